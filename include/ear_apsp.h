@@ -1,0 +1,195 @@
+/*
+ * ear_apsp.h -- C ABI of the B200-native ear-reduced all-pairs-shortest-paths library
+ * (libearapsp.so).  Paper: D. Dutta, M. Chaitanya, K. Kothapalli, D. Bera, "Applications of Ear
+ * Decomposition to Efficient Heterogeneous Algorithms for Shortest Path/Cycle Problems"
+ * (IPDPS-W 2017 / IJNC 8(1) 2018).  "P:NN" = line NN of the paper text.
+ *
+ * Problem (sec. 1, sec. 2.1.3): an undirected graph G = (V, E) with positive integer edge
+ * weights (W: E -> R+; integer reading C1 in DESIGN.md); output S[s,t] = weight of a shortest
+ * s-t path for every pair.  The library follows Algorithm 1 APSP(G):
+ *   Phase I   ear_decompose   G^r = Reduce(G)                       (Alg. 1 line 2)
+ *   Phase II  apsp_reduced    S^r = APSP(G^r), blocked min-plus FW (Alg. 1 lines 4-7; FW
+ *                             replaces the per-source Dijkstra -- same unique matrix, reading C10)
+ *   Phase III expand_ears     S from S^r by UPDATE_DISTANCE         (Alg. 1 lines 9-11)
+ *   apsp_full                 all three phases.
+ *
+ * Conventions (all functions):
+ *   - Plain C types only.  `stream` is a cudaStream_t passed as void* (NULL = legacy default stream).
+ *   - Pointers named d_* are DEVICE pointers on the current CUDA device, owned by the caller; h_* are
+ *     HOST pointers owned by the caller.  No function allocates or frees caller memory.  Plans and
+ *     communicators are owned by the library and released only by *_destroy.
+ *   - Vertex ids are 0..n-1 (the caller's order); every output is in the caller's order.
+ *   - int32 distances.  EAR_INF marks "unreachable" (reading C11); S[s,s] = 0; S is symmetric.
+ *   - Return value: EAR_OK or a negative ear_status_t; nothing throws.  ear_last_error() returns a
+ *     thread-local human-readable message for the last failure.
+ *   - Asynchronous on `stream` unless stated.  Kernel faults surface as EAR_ECUDA at the next
+ *     synchronising call.  A plan is not thread-safe; distinct plans are.
+ */
+#ifndef EAR_APSP_H
+#define EAR_APSP_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define EAR_INF 0x3FFFFFFF   /* unreachable; INF + INF does not overflow int32 */
+#define EAR_TILE 128         /* FW tile size B; reduced dimensions are padded to multiples of it */
+
+typedef enum {
+  EAR_OK = 0,
+  EAR_EINVAL = -1,         /* bad argument: n < 1, m < 0, id out of [0,n), weight < 1, bad range */
+  EAR_ENOMEM = -2,         /* device or host allocation failed */
+  EAR_ECUDA = -3,          /* CUDA runtime / kernel error */
+  EAR_ENCCL = -4,          /* NCCL error */
+  EAR_EOVERFLOW = -5,      /* (n-1) * max weight >= EAR_INF: distances might not fit */
+  EAR_EUNSUPPORTED = -6    /* unsupported configuration (e.g. misaligned pointer where required) */
+} ear_status_t;
+
+enum {
+  EAR_FLAG_NONE = 0,
+  EAR_FLAG_NO_CONTRACT = 1 /* every vertex is a terminal: direct blocked FW on G (cfg3 baseline) */
+};
+
+typedef struct ear_plan_s *ear_plan_t; /* Reduce(G) result: descriptors + reduced edge list (device) */
+typedef struct ear_comm_s *ear_comm_t; /* NCCL communicator for row-block sharding; NULL = 1 GPU */
+
+/* Summary of a plan.  n_reduced_padded depends on the number of ranks (padding to EAR_TILE*nranks). */
+typedef struct {
+  int32_t n;                /* |V| */
+  int32_t n_reduced;        /* |V^r| (vertices of degree != 2, plus one anchor per pure cycle) */
+  int32_t n_reduced_padded; /* Np: |V^r| rounded up to a multiple of EAR_TILE * nranks */
+  int32_t n_chains;         /* number of maximal degree-two chains (ears after reduction) */
+  int32_t max_chain_len;    /* most degree-two vertices on one chain */
+  int32_t n_promoted;       /* pure-cycle components whose min-id vertex became a terminal (C5) */
+  int64_t n_reduced_edges;  /* directed G^r arcs fed to D (both directions; before the P:90 min) */
+  int64_t m_simple;         /* undirected edges after dropping self-loops / merging parallels (C3) */
+  int32_t rank_rounds;      /* pointer-jumping rounds used by the chain ranking */
+  int32_t max_weight;       /* largest input weight */
+} ear_plan_info_t;
+
+/* ---------------------------------------------------------------- Phase I: Reduce(G)
+ * Alg. 1 line 2 "G^r = Reduce(G)"; the reduced graph of P:88 with the parallel-edge rule of
+ * P:90.  Input: m undirected edges (d_src[i], d_dst[i], d_w[i]), caller-owned DEVICE int32 arrays;
+ * either or both directions may be given; self-loops are ignored and parallel edges keep the
+ * minimum weight (reading C3).  Terminals (V^r) are vertices of degree != 2 (reading C4) plus the
+ * minimum-id vertex of every pure-cycle component (C5).  Every maximal chain of degree-two vertices
+ * becomes one G^r edge whose weight is the chain's weight sum; each chain vertex records its
+ * two chain ends (left/right), its along-chain distance to each (reading C7) and its chain
+ * (ear) id.  Terminal ids (tid) are assigned in increasing caller-id order.
+ * Synchronises `stream` (N_r is data dependent).  On success *out is a new plan (caller destroys it
+ * with ear_plan_destroy).  Errors: EAR_EINVAL (n < 1, m < 0, ids out of range, weight < 1),
+ * EAR_EOVERFLOW ((n-1)*max weight >= EAR_INF), EAR_ENOMEM, EAR_ECUDA. */
+ear_status_t ear_decompose(int32_t n, int64_t m, const int32_t *d_src, const int32_t *d_dst,
+                           const int32_t *d_w, uint32_t flags, void *stream, ear_plan_t *out);
+
+/* Plan summary for `nranks` ranks (1 for a single GPU).  Host-only, no synchronisation. */
+ear_status_t ear_plan_info(ear_plan_t plan, int32_t nranks, ear_plan_info_t *info);
+
+/* Copy the per-vertex descriptors to caller DEVICE arrays of n int32 each (any may be NULL):
+ * tid (terminal id or -1), ear (chain id or -1), left/right (tid of the chain ends; a terminal's own
+ * tid), off_left/off_right (along-chain distance to those ends; 0 for terminals).  For tests. */
+ear_status_t ear_plan_export(ear_plan_t plan, int32_t *d_tid, int32_t *d_ear, int32_t *d_left,
+                             int32_t *d_right, int32_t *d_off_left, int32_t *d_off_right, void *stream);
+
+/* Copy the directed G^r arcs (before the P:90 min; both directions) to caller DEVICE arrays of
+ * info.n_reduced_edges entries each: (tid u, tid v, weight).  For tests. */
+ear_status_t ear_plan_export_reduced_edges(ear_plan_t plan, int32_t *d_u, int32_t *d_v, int32_t *d_w,
+                                           void *stream);
+
+void ear_plan_destroy(ear_plan_t plan);
+
+/* ---------------------------------------------------------------- Phase II: APSP(G^r)
+ * Alg. 1 lines 4-7: D = S^r, all-pairs shortest paths on G^r, computed by a
+ * three-phase blocked min-plus Floyd-Warshall (prior art [23]) over EAR_TILE x EAR_TILE int32
+ * tiles; D is initialised here (EAR_INF, 0 diagonal, min over parallel G^r edges).
+ * Layout: row-major int32, leading dimension ldd (elements, ldd >= Np and ldd % 4 == 0, d_D 16-byte
+ * aligned), Np = info.n_reduced_padded; padded vertices are isolated.
+ *   comm == NULL: d_D is the full Np x Np matrix.
+ *   comm != NULL: d_D is this rank's row block, rows [rank*Np/P, (rank+1)*Np/P) x all Np columns
+ *                 (Np from ear_plan_info with nranks = P); the pivot row block is broadcast over
+ *                 NCCL each round.
+ * Asynchronous.  Errors: EAR_EINVAL (ldd too small/misaligned), EAR_ENCCL, EAR_ECUDA. */
+ear_status_t apsp_reduced(ear_plan_t plan, int32_t *d_D, int64_t ldd, ear_comm_t comm, void *stream);
+
+/* All-gather the row blocks produced by apsp_reduced with `comm` into the full Np x Np matrix
+ * d_D_full (ldd_full >= Np).  d_D_block may alias this rank's rows of d_D_full when
+ * ldd_block == ldd_full and d_D_block == d_D_full + rank*(Np/P)*ldd_full. */
+ear_status_t ear_gather_reduced(ear_plan_t plan, const int32_t *d_D_block, int64_t ldd_block,
+                                int32_t *d_D_full, int64_t ldd_full, ear_comm_t comm, void *stream);
+
+/* ---------------------------------------------------------------- Phase III: UPDATE_DISTANCE
+ * Alg. 1 lines 9-11 with the rules of sec. 2.1.3: for rows
+ * s in [row_begin, row_end) of S and every column t (caller order):
+ *   u, v in V^r                : S[u,v] = D[u,v]
+ *   x chain vertex, v in V^r   : S[x,v] = min(D[l_x,v] + wt(x,l_x), D[r_x,v] + wt(x,r_x))
+ *   x, y chain vertices        : 4-term minimum over {l_x,r_x} x {l_y,r_y}
+ *   x, y on the same chain     : also min with the along-chain distance |off_x - off_y|
+ *                                (same-ear test by chain id: readings C8, C9)
+ * then clamped to EAR_INF.  d_D_full is the FULL Np x Np matrix from apsp_reduced (ldd).  d_out is
+ * caller-owned (row_end - row_begin) x n int32, row-major with leading dimension ldo >= n.  The
+ * 128-bit store path is used when d_out is 16-byte aligned and ldo % 4 == 0 (otherwise a scalar
+ * path).  Asynchronous.  Errors: EAR_EINVAL (range, ldo < n, ldd), EAR_ECUDA. */
+ear_status_t expand_ears(ear_plan_t plan, const int32_t *d_D_full, int64_t ldd, int32_t row_begin,
+                         int32_t row_end, int32_t *d_out, int64_t ldo, void *stream);
+
+/* ---------------------------------------------------------------- Everything: Algorithm 1
+ * APSP(G): ear_decompose + apsp_reduced (+ all-gather with comm) + expand_ears into rows
+ * [row_begin, row_end) of S (d_out as in expand_ears).  Scratch (D) is allocated internally from
+ * the device heap and freed before return.  Synchronises `stream` once (inside ear_decompose) and
+ * again before freeing scratch.  With comm, each rank passes its own row range (ear_row_block). */
+ear_status_t apsp_full(int32_t n, int64_t m, const int32_t *d_src, const int32_t *d_dst,
+                       const int32_t *d_w, uint32_t flags, int32_t row_begin, int32_t row_end,
+                       int32_t *d_out, int64_t ldo, ear_comm_t comm, void *stream);
+
+/* Same as apsp_full with HOST input and output buffers (h_src/h_dst/h_w: m entries; h_out:
+ * (row_end-row_begin) x ldo).  Copies in, computes, copies the rows out (pinned h_out is fastest).
+ * Synchronous.  This is the end-to-end entry point bench.py times for its "e2e" figure. */
+ear_status_t apsp_full_host(int32_t n, int64_t m, const int32_t *h_src, const int32_t *h_dst,
+                            const int32_t *h_w, uint32_t flags, int32_t row_begin, int32_t row_end,
+                            int32_t *h_out, int64_t ldo, ear_comm_t comm, void *stream);
+
+/* ---------------------------------------------------------------- multi-GPU plumbing
+ * Contiguous near-equal split of `rows` rows over nranks: rank gets [*begin, *end). */
+void ear_row_block(int32_t rows, int32_t nranks, int32_t rank, int32_t *begin, int32_t *end);
+
+/* NCCL unique id (128 bytes) created on rank 0 and distributed by the caller (torch.distributed). */
+ear_status_t ear_comm_unique_id(uint8_t id[128]);
+/* Create this rank's communicator on the current CUDA device.  Collective over all ranks. */
+ear_status_t ear_comm_init(const uint8_t id[128], int32_t nranks, int32_t rank, ear_comm_t *out);
+ear_status_t ear_comm_info(ear_comm_t comm, int32_t *nranks, int32_t *rank);
+void ear_comm_destroy(ear_comm_t comm);
+
+/* ---------------------------------------------------------------- profiling (bench.py, tests)
+ * When enabled, CUDA events bracket every launch of the library's kernels on the stream they run on
+ * (a few microseconds per launch), and per-kernel-class device durations, launch counts and
+ * algorithmic work accumulate until ear_profile_reset.  Process-wide, not thread-safe. */
+typedef struct {
+  int64_t launches;            /* kernels of this library launched (counted whether or not enabled) */
+  double decompose_ms;         /* Phase I (ear_decompose), device time including its host syncs */
+  double fw_init_ms;           /* D initialisation */
+  double fw_phase1_ms, fw_phase2_ms, fw_phase3_ms;
+  int64_t fw_phase1_launches, fw_phase2_launches, fw_phase3_launches;
+  double fw_phase2_minplus;    /* algorithmic min-plus operations (one VIADDMNMX each) */
+  double fw_phase3_minplus;
+  double comm_ms;              /* pivot broadcasts + all-gather (multi-GPU) */
+  double expand_ms, same_chain_ms;
+  int64_t expand_launches;
+  double expand_bytes;         /* algorithmic HBM bytes of k_expand: 4*rows*n + 4*Nr^2 + 16*n */
+} ear_profile_t;
+
+void ear_profile_enable(int32_t on);
+void ear_profile_reset(void);
+/* Waits for the recorded events, folds them into *out (cumulative since the last reset). */
+ear_status_t ear_profile_read(ear_profile_t *out);
+
+/* ---------------------------------------------------------------- diagnostics */
+const char *ear_status_string(ear_status_t status);
+const char *ear_last_error(void);   /* thread-local; "" if none */
+const char *ear_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* EAR_APSP_H */

@@ -1,0 +1,318 @@
+// C-ABI entry points of libearapsp.so (declared and documented in include/ear_apsp.h).
+#include <cstdarg>
+#include <cstring>
+
+#include "common.cuh"
+
+namespace ear {
+
+static thread_local char g_err[512] = "";
+
+void set_error(const char *fmt, ...) {
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(g_err, sizeof(g_err), fmt, ap);
+  va_end(ap);
+}
+
+namespace {
+
+__global__ void k_export(int32_t n, const VDesc *desc, const int32_t *tidv, const int32_t *earv, int32_t *tid,
+                         int32_t *ear, int32_t *left, int32_t *right, int32_t *offl, int32_t *offr) {
+  for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
+    const VDesc d = desc[v];
+    if (tid) tid[v] = tidv[v];
+    if (ear) ear[v] = earv[v];
+    if (left) left[v] = d.p;
+    if (right) right[v] = d.q;
+    if (offl) offl[v] = d.cp;
+    if (offr) offr[v] = d.cq;
+  }
+}
+
+int32_t padded(const ear_plan_s *p, int32_t nranks) {
+  return (int32_t)round_up(std::max<int64_t>(p->n_reduced, 1), (int64_t)TILE * nranks);
+}
+
+bool aligned16(const void *p) { return ((uintptr_t)p & 15u) == 0; }
+
+}  // namespace
+}  // namespace ear
+
+using namespace ear;
+
+extern "C" {
+
+const char *ear_last_error(void) { return g_err; }
+
+const char *ear_version(void) { return "earapsp 0.1 (sm_100a)"; }
+
+const char *ear_status_string(ear_status_t s) {
+  switch (s) {
+    case EAR_OK: return "EAR_OK";
+    case EAR_EINVAL: return "EAR_EINVAL";
+    case EAR_ENOMEM: return "EAR_ENOMEM";
+    case EAR_ECUDA: return "EAR_ECUDA";
+    case EAR_ENCCL: return "EAR_ENCCL";
+    case EAR_EOVERFLOW: return "EAR_EOVERFLOW";
+    case EAR_EUNSUPPORTED: return "EAR_EUNSUPPORTED";
+  }
+  return "EAR_?";
+}
+
+void ear_row_block(int32_t rows, int32_t nranks, int32_t rank, int32_t *begin, int32_t *end) {
+  if (nranks < 1) nranks = 1;
+  if (begin) *begin = (int32_t)((int64_t)rows * rank / nranks);
+  if (end) *end = (int32_t)((int64_t)rows * (rank + 1) / nranks);
+}
+
+ear_status_t ear_decompose(int32_t n, int64_t m, const int32_t *d_src, const int32_t *d_dst, const int32_t *d_w,
+                           uint32_t flags, void *stream, ear_plan_t *out) {
+  g_err[0] = 0;
+  if (!out) { set_error("ear_decompose: out is NULL"); return EAR_EINVAL; }
+  *out = nullptr;
+  if (n < 1 || m < 0 || (m > 0 && (!d_src || !d_dst || !d_w)) || 2 * m > (int64_t)INT32_MAX) {
+    set_error("ear_decompose: bad sizes n=%d m=%lld", n, (long long)m);
+    return EAR_EINVAL;
+  }
+  ear_plan_s *p = new ear_plan_s;
+  cudaGetDevice(&p->device);
+  int sp = prof_begin(PK_DECOMPOSE, (cudaStream_t)stream);
+  ear_status_t s = decompose(n, m, d_src, d_dst, d_w, flags, (cudaStream_t)stream, p);
+  prof_end(sp, (cudaStream_t)stream, 0);
+  if (s != EAR_OK) {
+    cudaStreamSynchronize((cudaStream_t)stream);
+    plan_free(p);
+    delete p;
+    return s;
+  }
+  *out = p;
+  return EAR_OK;
+}
+
+ear_status_t ear_plan_info(ear_plan_t p, int32_t nranks, ear_plan_info_t *info) {
+  if (!p || !info || nranks < 1) { set_error("ear_plan_info: bad arguments"); return EAR_EINVAL; }
+  info->n = p->n;
+  info->n_reduced = p->n_reduced;
+  info->n_reduced_padded = padded(p, nranks);
+  info->n_chains = p->n_chains;
+  info->max_chain_len = p->max_chain_len;
+  info->n_promoted = p->n_promoted;
+  info->n_reduced_edges = p->n_redges;
+  info->m_simple = p->m_simple;
+  info->rank_rounds = p->rank_rounds;
+  info->max_weight = p->max_weight;
+  return EAR_OK;
+}
+
+ear_status_t ear_plan_export(ear_plan_t p, int32_t *d_tid, int32_t *d_ear, int32_t *d_left, int32_t *d_right,
+                             int32_t *d_off_left, int32_t *d_off_right, void *stream) {
+  if (!p) { set_error("ear_plan_export: NULL plan"); return EAR_EINVAL; }
+  int grid = (int)std::min<int64_t>(ceil_div(p->n, 256), 4096);
+  EAR_LAUNCH(k_export, grid, 256, 0, (cudaStream_t)stream)(p->n, p->desc, p->tid, p->ear, d_tid, d_ear, d_left, d_right,
+                                                    d_off_left, d_off_right);
+  EAR_CUDA_TRY(cudaGetLastError());
+  return EAR_OK;
+}
+
+ear_status_t ear_plan_export_reduced_edges(ear_plan_t p, int32_t *d_u, int32_t *d_v, int32_t *d_w, void *stream) {
+  if (!p) { set_error("ear_plan_export_reduced_edges: NULL plan"); return EAR_EINVAL; }
+  if (p->n_redges == 0) return EAR_OK;
+  cudaStream_t st = (cudaStream_t)stream;
+  size_t b = sizeof(int32_t) * (size_t)p->n_redges;
+  if (d_u) EAR_CUDA_TRY(cudaMemcpyAsync(d_u, p->re_u, b, cudaMemcpyDeviceToDevice, st));
+  if (d_v) EAR_CUDA_TRY(cudaMemcpyAsync(d_v, p->re_v, b, cudaMemcpyDeviceToDevice, st));
+  if (d_w) EAR_CUDA_TRY(cudaMemcpyAsync(d_w, p->re_w, b, cudaMemcpyDeviceToDevice, st));
+  return EAR_OK;
+}
+
+void ear_plan_destroy(ear_plan_t p) {
+  if (!p) return;
+  plan_free(p);
+  delete p;
+}
+
+ear_status_t apsp_reduced(ear_plan_t p, int32_t *d_D, int64_t ldd, ear_comm_t comm, void *stream) {
+  g_err[0] = 0;
+  if (!p || !d_D) { set_error("apsp_reduced: NULL argument"); return EAR_EINVAL; }
+  const int32_t P = comm ? comm->nranks : 1;
+  const int32_t Np = padded(p, P);
+  if (ldd < Np || ldd % 4 != 0 || !aligned16(d_D)) {
+    set_error("apsp_reduced: need ldd >= Np=%d, ldd %% 4 == 0 and a 16-byte aligned D (ldd=%lld)", Np,
+              (long long)ldd);
+    return EAR_EINVAL;
+  }
+  cudaStream_t st = (cudaStream_t)stream;
+  if (P == 1) {
+    EAR_TRY(fw_init_D(p, d_D, ldd, Np, 0, Np, st));
+    return fw_single(d_D, ldd, Np, st);
+  }
+  const int32_t rows = Np / P, row0 = comm->rank * rows;
+  EAR_TRY(fw_init_D(p, d_D, ldd, Np, row0, rows, st));
+  return fw_sharded(d_D, ldd, Np, comm, st);
+}
+
+ear_status_t ear_gather_reduced(ear_plan_t p, const int32_t *d_D_block, int64_t ldd_block, int32_t *d_D_full,
+                                int64_t ldd_full, ear_comm_t comm, void *stream) {
+  if (!p || !d_D_block || !d_D_full) { set_error("ear_gather_reduced: NULL argument"); return EAR_EINVAL; }
+  cudaStream_t st = (cudaStream_t)stream;
+  const int32_t P = comm ? comm->nranks : 1;
+  const int32_t Np = padded(p, P);
+  const int32_t rows = Np / P;
+  const int32_t rank = comm ? comm->rank : 0;
+  if (ldd_block < Np || ldd_full < Np) { set_error("ear_gather_reduced: leading dimension < Np"); return EAR_EINVAL; }
+  if (P == 1) {
+    if (d_D_block != d_D_full)
+      EAR_CUDA_TRY(cudaMemcpy2DAsync(d_D_full, sizeof(int32_t) * ldd_full, d_D_block, sizeof(int32_t) * ldd_block,
+                                     sizeof(int32_t) * Np, Np, cudaMemcpyDeviceToDevice, st));
+    return EAR_OK;
+  }
+  const int64_t cnt = (int64_t)rows * Np;
+  if (ldd_block == Np && ldd_full == Np) {
+    return comm_allgather(comm, d_D_block, d_D_full, cnt, st);
+  }
+  // general leading dimensions: pack, gather into a contiguous buffer, unpack
+  int32_t *tmp = nullptr;
+  EAR_CUDA_TRY(cudaMallocAsync((void **)&tmp, sizeof(int32_t) * (size_t)Np * Np, st));
+  EAR_CUDA_TRY(cudaMemcpy2DAsync(tmp + (int64_t)rank * cnt, sizeof(int32_t) * Np, d_D_block,
+                                 sizeof(int32_t) * ldd_block, sizeof(int32_t) * Np, rows, cudaMemcpyDeviceToDevice, st));
+  ear_status_t s = comm_allgather(comm, tmp + (int64_t)rank * cnt, tmp, cnt, st);
+  if (s == EAR_OK) {
+    cudaError_t e = cudaMemcpy2DAsync(d_D_full, sizeof(int32_t) * ldd_full, tmp, sizeof(int32_t) * Np,
+                                      sizeof(int32_t) * Np, Np, cudaMemcpyDeviceToDevice, st);
+    if (e != cudaSuccess) { set_error("gather unpack: %s", cudaGetErrorString(e)); s = EAR_ECUDA; }
+  }
+  cudaFreeAsync(tmp, st);
+  return s;
+}
+
+ear_status_t expand_ears(ear_plan_t p, const int32_t *d_D_full, int64_t ldd, int32_t row_begin, int32_t row_end,
+                         int32_t *d_out, int64_t ldo, void *stream) {
+  g_err[0] = 0;
+  if (!p || !d_D_full || (!d_out && row_end > row_begin)) { set_error("expand_ears: NULL argument"); return EAR_EINVAL; }
+  if (row_begin < 0 || row_end < row_begin || row_end > p->n || ldo < p->n || ldd < p->n_reduced) {
+    set_error("expand_ears: bad range [%d,%d) of n=%d or ldo=%lld / ldd=%lld too small", row_begin, row_end, p->n,
+              (long long)ldo, (long long)ldd);
+    return EAR_EINVAL;
+  }
+  return expand(p, d_D_full, ldd, row_begin, row_end, d_out, ldo, (cudaStream_t)stream);
+}
+
+// Phases II + III for an existing plan into device rows (shared by apsp_full / apsp_full_host).
+static ear_status_t solve_rows(ear_plan_s *p, int32_t row_begin, int32_t row_end, int32_t *d_out, int64_t ldo,
+                               ear_comm_t comm, cudaStream_t st, int32_t **D_keep) {
+  const int32_t P = comm ? comm->nranks : 1;
+  const int32_t Np = padded(p, P);
+  int32_t *D = nullptr, *Dfull = nullptr;
+  ear_status_t s = EAR_OK;
+  if (P == 1) {
+    EAR_CUDA_TRY(cudaMallocAsync((void **)&D, sizeof(int32_t) * (size_t)Np * Np, st));
+    s = apsp_reduced(p, D, Np, nullptr, st);
+    Dfull = D;
+  } else {
+    EAR_CUDA_TRY(cudaMallocAsync((void **)&Dfull, sizeof(int32_t) * (size_t)Np * Np, st));
+    D = Dfull + (int64_t)comm->rank * (Np / P) * Np;   // this rank's rows, in place
+    s = apsp_reduced(p, D, Np, comm, st);
+    if (s == EAR_OK) s = ear_gather_reduced(p, D, Np, Dfull, Np, comm, st);
+  }
+  if (s == EAR_OK && d_out) s = expand_ears(p, Dfull, Np, row_begin, row_end, d_out, ldo, st);
+  if (D_keep && s == EAR_OK) {
+    *D_keep = Dfull;
+  } else {
+    cudaFreeAsync(Dfull, st);
+  }
+  return s;
+}
+
+ear_status_t apsp_full(int32_t n, int64_t m, const int32_t *d_src, const int32_t *d_dst, const int32_t *d_w,
+                       uint32_t flags, int32_t row_begin, int32_t row_end, int32_t *d_out, int64_t ldo,
+                       ear_comm_t comm, void *stream) {
+  cudaStream_t st = (cudaStream_t)stream;
+  if (row_begin < 0 || row_end < row_begin || row_end > n || ldo < n) {
+    set_error("apsp_full: bad row range [%d,%d) or ldo=%lld for n=%d", row_begin, row_end, (long long)ldo, n);
+    return EAR_EINVAL;
+  }
+  ear_plan_t p = nullptr;
+  EAR_TRY(ear_decompose(n, m, d_src, d_dst, d_w, flags, stream, &p));
+  ear_status_t s = solve_rows(p, row_begin, row_end, d_out, ldo, comm, st, nullptr);
+  cudaError_t e = cudaStreamSynchronize(st);
+  ear_plan_destroy(p);
+  if (s == EAR_OK && e != cudaSuccess) {
+    set_error("apsp_full: %s", cudaGetErrorString(e));
+    s = EAR_ECUDA;
+  }
+  return s;
+}
+
+ear_status_t apsp_full_host(int32_t n, int64_t m, const int32_t *h_src, const int32_t *h_dst, const int32_t *h_w,
+                            uint32_t flags, int32_t row_begin, int32_t row_end, int32_t *h_out, int64_t ldo,
+                            ear_comm_t comm, void *stream) {
+  cudaStream_t st = (cudaStream_t)stream;
+  if (row_begin < 0 || row_end < row_begin || row_end > n || ldo < n || (m > 0 && (!h_src || !h_dst || !h_w))) {
+    set_error("apsp_full_host: bad arguments");
+    return EAR_EINVAL;
+  }
+  // 1. edges host -> device
+  int32_t *dE = nullptr;
+  const size_t eb = sizeof(int32_t) * (size_t)std::max<int64_t>(m, 1);
+  EAR_CUDA_TRY(cudaMallocAsync((void **)&dE, 3 * eb, st));
+  if (m > 0) {
+    EAR_CUDA_TRY(cudaMemcpyAsync(dE, h_src, eb, cudaMemcpyHostToDevice, st));
+    EAR_CUDA_TRY(cudaMemcpyAsync(dE + m, h_dst, eb, cudaMemcpyHostToDevice, st));
+    EAR_CUDA_TRY(cudaMemcpyAsync(dE + 2 * m, h_w, eb, cudaMemcpyHostToDevice, st));
+  }
+  ear_plan_t p = nullptr;
+  ear_status_t s = ear_decompose(n, m, dE, dE + m, dE + 2 * m, flags, stream, &p);
+  cudaFreeAsync(dE, st);
+  if (s != EAR_OK) return s;
+  // 2. reduced APSP, D kept
+  int32_t *Dfull = nullptr;
+  s = solve_rows(p, row_begin, row_end, nullptr, ldo, comm, st, &Dfull);
+  const int32_t P = comm ? comm->nranks : 1;
+  const int32_t Np = padded(p, P);
+  // 3. expansion in row chunks, double-buffered against the device -> host copies
+  const int32_t rows = row_end - row_begin;
+  if (s == EAR_OK && rows > 0) {
+    int32_t chunk = (int32_t)std::max<int64_t>(32, std::min<int64_t>(rows, (256ll << 20) / (4ll * n)));
+    chunk = (int32_t)round_up(chunk, 32);
+    int32_t *buf[2] = {nullptr, nullptr};
+    cudaStream_t cs = nullptr;
+    cudaEvent_t ready[2] = {nullptr, nullptr}, freed[2] = {nullptr, nullptr};
+    cudaError_t e = cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking);
+    for (int i = 0; i < 2 && e == cudaSuccess; ++i) {
+      e = cudaMallocAsync((void **)&buf[i], sizeof(int32_t) * (size_t)chunk * n, st);
+      if (e == cudaSuccess) e = cudaEventCreateWithFlags(&ready[i], cudaEventDisableTiming);
+      if (e == cudaSuccess) e = cudaEventCreateWithFlags(&freed[i], cudaEventDisableTiming);
+    }
+    if (e != cudaSuccess) { set_error("apsp_full_host: %s", cudaGetErrorString(e)); s = EAR_ECUDA; }
+    int it = 0;
+    for (int32_t r = row_begin; s == EAR_OK && r < row_end; r += chunk, ++it) {
+      const int b = it & 1;
+      const int32_t r1 = std::min(row_end, r + chunk);
+      if (it >= 2) cudaStreamWaitEvent(st, freed[b], 0);
+      s = expand(p, Dfull, Np, r, r1, buf[b], n, st);
+      if (s != EAR_OK) break;
+      cudaEventRecord(ready[b], st);
+      cudaStreamWaitEvent(cs, ready[b], 0);
+      e = cudaMemcpy2DAsync(h_out + (int64_t)(r - row_begin) * ldo, sizeof(int32_t) * ldo, buf[b],
+                            sizeof(int32_t) * n, sizeof(int32_t) * n, r1 - r, cudaMemcpyDeviceToHost, cs);
+      if (e != cudaSuccess) { set_error("apsp_full_host D2H: %s", cudaGetErrorString(e)); s = EAR_ECUDA; break; }
+      cudaEventRecord(freed[b], cs);
+    }
+    cudaStreamSynchronize(cs);
+    cudaStreamSynchronize(st);
+    for (int i = 0; i < 2; ++i) {
+      if (buf[i]) cudaFreeAsync(buf[i], st);
+      if (ready[i]) cudaEventDestroy(ready[i]);
+      if (freed[i]) cudaEventDestroy(freed[i]);
+    }
+    if (cs) cudaStreamDestroy(cs);
+  }
+  if (Dfull) cudaFreeAsync(Dfull, st);
+  cudaError_t e = cudaStreamSynchronize(st);
+  ear_plan_destroy(p);
+  if (s == EAR_OK && e != cudaSuccess) { set_error("apsp_full_host: %s", cudaGetErrorString(e)); s = EAR_ECUDA; }
+  return s;
+}
+
+}  // extern "C"

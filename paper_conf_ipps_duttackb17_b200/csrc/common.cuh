@@ -1,0 +1,101 @@
+// Shared internals of libearapsp.so (product path only; nothing here is shared with oracle/).
+#pragma once
+#include <cstdint>
+#include <cstdio>
+#include <cuda_runtime.h>
+
+#include "ear_apsp.h"
+
+namespace ear {
+
+constexpr int TILE = EAR_TILE;   // FW tile (B)
+constexpr int32_t INF = EAR_INF;
+
+// thread-local last-error text
+void set_error(const char *fmt, ...);
+
+#define EAR_CUDA_TRY(expr)                                                                   \
+  do {                                                                                       \
+    cudaError_t _e = (expr);                                                                 \
+    if (_e != cudaSuccess) {                                                                 \
+      ::ear::set_error("%s:%d %s: %s", __FILE__, __LINE__, #expr, cudaGetErrorString(_e));   \
+      return EAR_ECUDA;                                                                      \
+    }                                                                                        \
+  } while (0)
+
+#define EAR_TRY(expr)                  \
+  do {                                 \
+    ear_status_t _s = (expr);          \
+    if (_s != EAR_OK) return _s;       \
+  } while (0)
+
+inline int64_t ceil_div(int64_t a, int64_t b) { return (a + b - 1) / b; }
+inline int64_t round_up(int64_t a, int64_t b) { return ceil_div(a, b) * b; }
+
+// Per-vertex expansion descriptor (16 B): p = tid(left end), cp = along-chain distance to it,
+// q = tid(right end), cq = distance to it.  Terminals: p = q = own tid, cp = cq = 0.
+struct __align__(16) VDesc {
+  int32_t p, cp, q, cq;
+};
+
+}  // namespace ear
+
+// Library-owned plan (Reduce(G) result), device arrays unless noted.
+struct ear_plan_s {
+  int32_t n = 0;
+  int32_t n_reduced = 0;
+  int32_t n_chains = 0;
+  int32_t max_chain_len = 0;
+  int32_t n_promoted = 0;
+  int32_t rank_rounds = 0;
+  int32_t max_weight = 0;
+  int64_t m_simple = 0;
+  int64_t n_redges = 0;
+  uint32_t flags = 0;
+  int device = 0;
+  // per vertex
+  ear::VDesc *desc = nullptr;  // [n]
+  int32_t *tid = nullptr;      // [n] terminal id or -1
+  int32_t *ear = nullptr;      // [n] chain id or -1
+  // same-ear patch structure: chain vertices grouped by chain, sorted by off_left
+  int32_t *seg_of = nullptr;    // [n] segment (chain) index of a chain vertex, -1 for terminals
+  int32_t *seg_start = nullptr; // [n_chains + 1]
+  int32_t *seg_vert = nullptr;  // [#chain vertices]
+  int32_t n_chain_vertices = 0;
+  // reduced arcs (both directions, before the P:90 min)
+  int32_t *re_u = nullptr, *re_v = nullptr, *re_w = nullptr;
+};
+
+struct ear_comm_s {
+  void *nccl = nullptr;  // ncclComm_t
+  int32_t nranks = 1;
+  int32_t rank = 0;
+  int device = 0;
+  cudaStream_t comm_stream = nullptr;
+};
+
+namespace ear {
+// prof.cu
+enum ProfKind { PK_DECOMPOSE, PK_FW_INIT, PK_FW_P1, PK_FW_P2, PK_FW_P3, PK_COMM, PK_EXPAND, PK_SAME_CHAIN };
+void count_launch(int n = 1);
+int prof_begin(int kind, cudaStream_t s);                // -1 when profiling is off
+void prof_end(int slot, cudaStream_t s, double work);
+// launch one of the library's kernels and count it: EAR_LAUNCH(k, grid, block, smem, stream)(args);
+#define EAR_LAUNCH(k, g, b, sm, st) ::ear::count_launch(), k<<<(g), (b), (sm), (st)>>>
+// decompose.cu
+ear_status_t decompose(int32_t n, int64_t m, const int32_t *src, const int32_t *dst, const int32_t *w,
+                       uint32_t flags, cudaStream_t stream, ear_plan_s *plan);
+void plan_free(ear_plan_s *plan);
+// fw.cu
+ear_status_t fw_init_D(const ear_plan_s *plan, int32_t *D, int64_t ldd, int32_t Np, int32_t row0,
+                       int32_t rows, cudaStream_t stream);
+ear_status_t fw_single(int32_t *D, int64_t ldd, int32_t Np, cudaStream_t stream);
+ear_status_t fw_sharded(int32_t *Dblk, int64_t ldd, int32_t Np, ear_comm_s *comm, cudaStream_t stream);
+// expand.cu
+ear_status_t expand(const ear_plan_s *plan, const int32_t *D, int64_t ldd, int32_t row_begin,
+                    int32_t row_end, int32_t *out, int64_t ldo, cudaStream_t stream);
+// comm.cu
+ear_status_t comm_bcast(ear_comm_s *comm, int32_t *buf, int64_t count, int32_t root, cudaStream_t stream);
+ear_status_t comm_allgather(ear_comm_s *comm, const int32_t *send, int32_t *recv, int64_t count,
+                            cudaStream_t stream);
+}  // namespace ear

@@ -1,0 +1,362 @@
+// Phase II -- S^r = APSP(G^r) (Alg. 1 lines 4-7) as a three-phase blocked min-plus
+// Floyd-Warshall (blocked FW of [23], cited at P:60) over 128 x 128 int32 tiles on sm_100a.
+//
+//   D init   INF everywhere, 0 on the diagonal, atomicMin of the G^r arcs (keep the shortest of
+//            parallel edges).
+//   round k  phase 1  closure of the pivot tile (k,k): serial kk loop in one CTA; the matrix is
+//                     symmetric (undirected G), so row kk doubles as column kk and one smem row
+//                     buffer (double-buffered) broadcasts the pivot each step;
+//            phase 2  pivot-row tiles (k,j): C = min(C, P (x) C) with the CLOSED pivot P -- a single
+//                     min-plus product, no serial dependency (closure argument in DESIGN.md);
+//            phase 3  remaining tiles (i,j): C = min(C, D[i,K] (x) D[K,j]).
+//   Both phase 2 and 3 run the same register-blocked min-plus tile kernel: 256 threads, 8x8 int32
+//   accumulators per thread, operands streamed through double-buffered shared memory by cp.async in
+//   32-deep k-chunks; one VIADDMNMX (c = min(c, a + b)) per min-plus.  Because D is symmetric,
+//   D[i,K] = D[K,i]^T: both operands are slices of the pivot ROW block, which is also the only
+//   block a multi-GPU round has to broadcast.  On one GPU only the upper triangle of tiles is
+//   computed and each result is written twice (tile and transposed mirror): half the min-plus work.
+#include <algorithm>
+#include <cmath>
+
+#include "common.cuh"
+
+namespace ear {
+namespace {
+
+constexpr int NT = 256;
+constexpr int KC = 32;                       // k-chunk depth
+constexpr int NCHUNK = TILE / KC;            // 4
+constexpr int SM_CHUNK = KC * TILE;          // ints per operand chunk (16 KB)
+constexpr int FW_SMEM = 2 * 2 * SM_CHUNK * 4; // 2 stages x 2 operands = 64 KB
+
+__global__ void k_init_D(int32_t *D, int64_t ldd, int32_t Np, int32_t row0, int32_t rows) {
+  int64_t total = (int64_t)rows * (Np / 4);
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
+    int32_t r = (int32_t)(i / (Np / 4));
+    int32_t c4 = (int32_t)(i % (Np / 4)) * 4;
+    int4 v = make_int4(INF, INF, INF, INF);
+    int32_t g = row0 + r;   // global row
+    if (g >= c4 && g < c4 + 4) ((int32_t *)&v)[g - c4] = 0;
+    *reinterpret_cast<int4 *>(D + (int64_t)r * ldd + c4) = v;
+  }
+}
+
+__global__ void k_init_edges(const int32_t *ru, const int32_t *rv, const int32_t *rw, int64_t E, int32_t *D,
+                             int64_t ldd, int32_t row0, int32_t rows) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < E; i += (int64_t)gridDim.x * blockDim.x) {
+    int32_t u = ru[i] - row0;
+    if (u >= 0 && u < rows) atomicMin(D + (int64_t)u * ldd + rv[i], rw[i]);
+  }
+}
+
+__device__ __forceinline__ int32_t mp(int32_t a, int32_t b, int32_t c) { return __viaddmin_s32(a, b, c); }
+
+// ------------------------------------------------------------------------------ phase 1
+// Closure of the 128x128 pivot tile at T (leading dimension ldt), in place.
+__global__ void __launch_bounds__(NT, 1) k_fw_phase1(int32_t *T, int64_t ldt) {
+  __shared__ __align__(16) int32_t rowbuf[2][TILE];
+  const int tx = threadIdx.x & 15, ty = threadIdx.x >> 4;
+  int32_t c[8][8];
+#pragma unroll
+  for (int r = 0; r < 8; ++r) {
+    const int i = (r < 4 ? 0 : 64) + ty * 4 + (r & 3);
+    const int4 lo = *reinterpret_cast<const int4 *>(T + (int64_t)i * ldt + tx * 4);
+    const int4 hi = *reinterpret_cast<const int4 *>(T + (int64_t)i * ldt + 64 + tx * 4);
+    c[r][0] = lo.x; c[r][1] = lo.y; c[r][2] = lo.z; c[r][3] = lo.w;
+    c[r][4] = hi.x; c[r][5] = hi.y; c[r][6] = hi.z; c[r][7] = hi.w;
+  }
+  // row 0 is owned by ty = 0, r = 0
+  if (ty == 0) {
+    *reinterpret_cast<int4 *>(&rowbuf[0][tx * 4]) = make_int4(c[0][0], c[0][1], c[0][2], c[0][3]);
+    *reinterpret_cast<int4 *>(&rowbuf[0][64 + tx * 4]) = make_int4(c[0][4], c[0][5], c[0][6], c[0][7]);
+  }
+  __syncthreads();
+  for (int kk = 0; kk < TILE; ++kk) {
+    const int32_t *rb = rowbuf[kk & 1];
+    const int4 alo = *reinterpret_cast<const int4 *>(rb + ty * 4);
+    const int4 ahi = *reinterpret_cast<const int4 *>(rb + 64 + ty * 4);
+    const int4 blo = *reinterpret_cast<const int4 *>(rb + tx * 4);
+    const int4 bhi = *reinterpret_cast<const int4 *>(rb + 64 + tx * 4);
+    const int32_t a[8] = {alo.x, alo.y, alo.z, alo.w, ahi.x, ahi.y, ahi.z, ahi.w};
+    const int32_t b[8] = {blo.x, blo.y, blo.z, blo.w, bhi.x, bhi.y, bhi.z, bhi.w};
+#pragma unroll
+    for (int r = 0; r < 8; ++r)
+#pragma unroll
+      for (int q = 0; q < 8; ++q) c[r][q] = mp(a[r], b[q], c[r][q]);
+    // publish row kk+1 (after this step's update) for the next step
+    const int nk = kk + 1;
+    if (nk < TILE && ty == ((nk & 63) >> 2)) {
+      const int rr = (nk & 3) + (nk >= 64 ? 4 : 0);
+      int32_t *wb = rowbuf[nk & 1];
+#pragma unroll
+      for (int r = 0; r < 8; ++r) {
+        if (r == rr) {
+          *reinterpret_cast<int4 *>(wb + tx * 4) = make_int4(c[r][0], c[r][1], c[r][2], c[r][3]);
+          *reinterpret_cast<int4 *>(wb + 64 + tx * 4) = make_int4(c[r][4], c[r][5], c[r][6], c[r][7]);
+        }
+      }
+    }
+    __syncthreads();
+  }
+#pragma unroll
+  for (int r = 0; r < 8; ++r) {
+    const int i = (r < 4 ? 0 : 64) + ty * 4 + (r & 3);
+    *reinterpret_cast<int4 *>(T + (int64_t)i * ldt + tx * 4) = make_int4(c[r][0], c[r][1], c[r][2], c[r][3]);
+    *reinterpret_cast<int4 *>(T + (int64_t)i * ldt + 64 + tx * 4) = make_int4(c[r][4], c[r][5], c[r][6], c[r][7]);
+  }
+}
+
+// ------------------------------------------------------------------------------ phases 2 and 3
+enum { MODE_PIVOT_ROW = 0, MODE_UPPER = 1, MODE_ROWS = 2 };
+
+struct TileJob {
+  int32_t *C;        // matrix holding the C tiles (local rows), leading dimension ldc
+  int64_t ldc;
+  const int32_t *P;  // pivot row block: 128 rows x Np, leading dimension ldp
+  int64_t ldp;
+  int32_t k;         // pivot tile index
+  int32_t nt;        // tiles per dimension (Np / 128)
+  int32_t ti0;       // first local tile row (global index) of C
+  int32_t nti;       // number of local tile rows
+  int32_t mode;
+  int32_t mirror;    // also write the transposed result into tile (tj, ti) (single GPU)
+};
+
+__device__ __forceinline__ void cp_async16(void *smem, const void *gmem) {
+  unsigned s = (unsigned)__cvta_generic_to_shared(smem);
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(s), "l"(gmem));
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;\n" ::"n"(N)); }
+
+// decode the CTA index into (ti, tj)
+__device__ __forceinline__ bool decode_tile(const TileJob &J, int64_t idx, int &ti, int &tj) {
+  const int k = J.k;
+  if (J.mode == MODE_PIVOT_ROW) {
+    ti = k;
+    tj = (int)idx < k ? (int)idx : (int)idx + 1;
+    return true;
+  }
+  if (J.mode == MODE_UPPER) {
+    // upper triangle (a <= b) of the (nt-1) x (nt-1) non-pivot tiles, row-major
+    const int64_t T = J.nt - 1;
+    // a = largest a with a*T - a*(a-1)/2 <= idx
+    double tt = (double)(2 * T + 1);
+    int64_t a = (int64_t)floor((tt - sqrt(tt * tt - 8.0 * (double)idx)) * 0.5);
+    if (a < 0) a = 0;
+    while (a > 0 && a * T - a * (a - 1) / 2 > idx) --a;
+    while ((a + 1) * T - (a + 1) * a / 2 <= idx) ++a;
+    const int64_t b = a + (idx - (a * T - a * (a - 1) / 2));
+    ti = (int)a < k ? (int)a : (int)a + 1;
+    tj = (int)b < k ? (int)b : (int)b + 1;
+    return true;
+  }
+  // MODE_ROWS: local tile rows except the pivot row, all columns except the pivot column
+  const int64_t ncols = J.nt - 1;
+  int r = (int)(idx / ncols), cidx = (int)(idx % ncols);
+  ti = J.ti0 + r;
+  if (ti >= k && k >= J.ti0 && k < J.ti0 + J.nti) ti++;   // skip the pivot tile row if local
+  tj = cidx < k ? cidx : cidx + 1;
+  return true;
+}
+
+__global__ void __launch_bounds__(NT, 2) k_fw_tiles(TileJob J) {
+  extern __shared__ __align__(16) int32_t smem[];
+  int32_t *sA = smem;                       // [2][KC][TILE]   A^T chunk = P[k-rows][ti cols]
+  int32_t *sB = smem + 2 * SM_CHUNK;        // [2][KC][TILE]   B chunk   = P[k-rows][tj cols]
+  const int tid = threadIdx.x;
+  const int tx = tid & 15, ty = tid >> 4;
+  int ti, tj;
+  decode_tile(J, blockIdx.x, ti, tj);
+
+  const int32_t *pa = J.P + (int64_t)ti * TILE;
+  const int32_t *pb = J.P + (int64_t)tj * TILE;
+  auto load_chunk = [&](int kc, int stage) {
+#pragma unroll
+    for (int it = 0; it < 4; ++it) {
+      const int piece = tid + it * NT;           // 0..1023: 32 rows x 32 pieces of 16 B
+      const int rr = piece >> 5, cc = (piece & 31) * 4;
+      const int64_t goff = (int64_t)(kc * KC + rr) * J.ldp + cc;
+      cp_async16(sA + stage * SM_CHUNK + rr * TILE + cc, pa + goff);
+      cp_async16(sB + stage * SM_CHUNK + rr * TILE + cc, pb + goff);
+    }
+    cp_async_commit();
+  };
+  load_chunk(0, 0);
+
+  // C tile -> registers
+  int32_t *Ct = J.C + (int64_t)(ti - J.ti0) * TILE * J.ldc + (int64_t)tj * TILE;
+  int32_t c[8][8];
+#pragma unroll
+  for (int r = 0; r < 8; ++r) {
+    const int i = (r < 4 ? 0 : 64) + ty * 4 + (r & 3);
+    const int4 lo = *reinterpret_cast<const int4 *>(Ct + (int64_t)i * J.ldc + tx * 4);
+    const int4 hi = *reinterpret_cast<const int4 *>(Ct + (int64_t)i * J.ldc + 64 + tx * 4);
+    c[r][0] = lo.x; c[r][1] = lo.y; c[r][2] = lo.z; c[r][3] = lo.w;
+    c[r][4] = hi.x; c[r][5] = hi.y; c[r][6] = hi.z; c[r][7] = hi.w;
+  }
+
+#pragma unroll 1
+  for (int kc = 0; kc < NCHUNK; ++kc) {
+    const int stage = kc & 1;
+    if (kc + 1 < NCHUNK) {
+      load_chunk(kc + 1, stage ^ 1);
+      cp_async_wait<1>();
+    } else {
+      cp_async_wait<0>();
+    }
+    __syncthreads();
+    const int32_t *a_s = sA + stage * SM_CHUNK;
+    const int32_t *b_s = sB + stage * SM_CHUNK;
+#pragma unroll 4
+    for (int kk = 0; kk < KC; ++kk) {
+      const int4 alo = *reinterpret_cast<const int4 *>(a_s + kk * TILE + ty * 4);
+      const int4 ahi = *reinterpret_cast<const int4 *>(a_s + kk * TILE + 64 + ty * 4);
+      const int4 blo = *reinterpret_cast<const int4 *>(b_s + kk * TILE + tx * 4);
+      const int4 bhi = *reinterpret_cast<const int4 *>(b_s + kk * TILE + 64 + tx * 4);
+      const int32_t a[8] = {alo.x, alo.y, alo.z, alo.w, ahi.x, ahi.y, ahi.z, ahi.w};
+      const int32_t b[8] = {blo.x, blo.y, blo.z, blo.w, bhi.x, bhi.y, bhi.z, bhi.w};
+#pragma unroll
+      for (int r = 0; r < 8; ++r)
+#pragma unroll
+        for (int q = 0; q < 8; ++q) c[r][q] = mp(a[r], b[q], c[r][q]);
+    }
+    __syncthreads();
+  }
+
+  // epilogue: tile, and (single GPU, off-diagonal) its transposed mirror
+#pragma unroll
+  for (int r = 0; r < 8; ++r) {
+    const int i = (r < 4 ? 0 : 64) + ty * 4 + (r & 3);
+    *reinterpret_cast<int4 *>(Ct + (int64_t)i * J.ldc + tx * 4) = make_int4(c[r][0], c[r][1], c[r][2], c[r][3]);
+    *reinterpret_cast<int4 *>(Ct + (int64_t)i * J.ldc + 64 + tx * 4) = make_int4(c[r][4], c[r][5], c[r][6], c[r][7]);
+  }
+  if (J.mirror && ti != tj) {
+    int32_t *Mt = J.C + (int64_t)tj * TILE * J.ldc + (int64_t)ti * TILE;
+#pragma unroll
+    for (int q = 0; q < 8; ++q) {
+      const int j = (q < 4 ? 0 : 64) + tx * 4 + (q & 3);
+      *reinterpret_cast<int4 *>(Mt + (int64_t)j * J.ldc + ty * 4) = make_int4(c[0][q], c[1][q], c[2][q], c[3][q]);
+      *reinterpret_cast<int4 *>(Mt + (int64_t)j * J.ldc + 64 + ty * 4) = make_int4(c[4][q], c[5][q], c[6][q], c[7][q]);
+    }
+  }
+}
+
+// transposed copy of the pivot row block's slice into this rank's column tiles (i, k):
+// D[i-block rows][k-block cols] = P[0..128)[i-block]^T  (phase 2 columns by symmetry)
+__global__ void k_col_tiles_from_pivot(int32_t *C, int64_t ldc, const int32_t *P, int64_t ldp, int32_t k,
+                                       int32_t ti0, int32_t nti) {
+  __shared__ int32_t t[32][33];
+  const int tile = blockIdx.y;                 // local tile row
+  const int ti = ti0 + tile;
+  if (ti == k) return;
+  const int bx = blockIdx.x & 3, by = blockIdx.x >> 2;  // 4 x 4 sub-blocks of 32 x 32
+  const int lx = threadIdx.x & 31, ly = threadIdx.x >> 5;  // 32 x 8
+  for (int yy = ly; yy < 32; yy += 8)   // P rows (k-local) by*32+yy, cols ti*128 + bx*32 + lx
+    t[yy][lx] = P[(int64_t)(by * 32 + yy) * ldp + (int64_t)ti * TILE + bx * 32 + lx];
+  __syncthreads();
+  for (int yy = ly; yy < 32; yy += 8)   // C rows (tile-local) bx*32+yy, cols k*128 + by*32 + lx
+    C[(int64_t)(tile * TILE + bx * 32 + yy) * ldc + (int64_t)k * TILE + by * 32 + lx] = t[lx][yy];
+}
+
+bool g_smem_set = false;
+
+ear_status_t launch_tiles(const TileJob &J, int64_t nblocks, cudaStream_t st) {
+  if (!g_smem_set) {
+    EAR_CUDA_TRY(cudaFuncSetAttribute(k_fw_tiles, cudaFuncAttributeMaxDynamicSharedMemorySize, FW_SMEM));
+    g_smem_set = true;
+  }
+  if (nblocks <= 0) return EAR_OK;
+  EAR_LAUNCH(k_fw_tiles, (unsigned)nblocks, NT, FW_SMEM, st)(J);
+  return EAR_OK;
+}
+
+}  // namespace
+
+ear_status_t fw_init_D(const ear_plan_s *plan, int32_t *D, int64_t ldd, int32_t Np, int32_t row0, int32_t rows,
+                       cudaStream_t st) {
+  int64_t total = (int64_t)rows * (Np / 4);
+  int grid = (int)std::min<int64_t>(ceil_div(total, 256), 148 * 32);
+  int s0 = prof_begin(PK_FW_INIT, st);
+  if (total > 0) EAR_LAUNCH(k_init_D, grid, 256, 0, st)(D, ldd, Np, row0, rows);
+  if (plan->n_redges > 0) {
+    int g2 = (int)std::min<int64_t>(ceil_div(plan->n_redges, 256), 148 * 32);
+    EAR_LAUNCH(k_init_edges, g2, 256, 0, st)(plan->re_u, plan->re_v, plan->re_w, plan->n_redges, D, ldd, row0, rows);
+  }
+  prof_end(s0, st, 0);
+  EAR_CUDA_TRY(cudaGetLastError());
+  return EAR_OK;
+}
+
+// Single GPU: full symmetric D (Np x Np).
+ear_status_t fw_single(int32_t *D, int64_t ldd, int32_t Np, cudaStream_t st) {
+  const int nt = Np / TILE;
+  const double tile_ops = (double)TILE * TILE * TILE;
+  for (int k = 0; k < nt; ++k) {
+    int32_t *Pk = D + (int64_t)k * TILE * ldd;            // pivot row block
+    int s1 = prof_begin(PK_FW_P1, st);
+    EAR_LAUNCH(k_fw_phase1, 1, NT, 0, st)(Pk + (int64_t)k * TILE, ldd);
+    prof_end(s1, st, tile_ops);
+    TileJob J{D, ldd, Pk, ldd, k, nt, 0, nt, MODE_PIVOT_ROW, 1};
+    int s2 = prof_begin(PK_FW_P2, st);
+    EAR_TRY(launch_tiles(J, nt - 1, st));
+    prof_end(s2, st, (nt - 1) * tile_ops);
+    J.mode = MODE_UPPER;
+    const int64_t nup = (int64_t)(nt - 1) * nt / 2;
+    int s3 = prof_begin(PK_FW_P3, st);
+    EAR_TRY(launch_tiles(J, nup, st));
+    prof_end(s3, st, nup * tile_ops);
+  }
+  EAR_CUDA_TRY(cudaGetLastError());
+  return EAR_OK;
+}
+
+// Row-block sharded: this rank holds rows [rank*R, (rank+1)*R) of D (R = Np / nranks, a multiple
+// of 128) in Dblk (leading dimension ldd).  Each round the owner of pivot block k closes the pivot
+// tile and its pivot-row tiles, the 128 x Np pivot row block is broadcast (NCCL), every rank fills
+// its column tiles by symmetry and updates its remaining tiles.
+ear_status_t fw_sharded(int32_t *Dblk, int64_t ldd, int32_t Np, ear_comm_s *comm, cudaStream_t st) {
+  const int nt = Np / TILE;
+  const int P = comm->nranks, rank = comm->rank;
+  const int nti = nt / P, ti0 = rank * nti;
+  const double tile_ops = (double)TILE * TILE * TILE;
+  int32_t *prow = nullptr;
+  EAR_CUDA_TRY(cudaMallocAsync((void **)&prow, sizeof(int32_t) * (size_t)TILE * Np, st));
+  ear_status_t status = EAR_OK;
+  for (int k = 0; k < nt && status == EAR_OK; ++k) {
+    const int owner = k / nti;
+    if (owner == rank) {
+      int32_t *Pk = Dblk + (int64_t)(k - ti0) * TILE * ldd;
+      int s1 = prof_begin(PK_FW_P1, st);
+      EAR_LAUNCH(k_fw_phase1, 1, NT, 0, st)(Pk + (int64_t)k * TILE, ldd);
+      prof_end(s1, st, tile_ops);
+      TileJob J{Pk, ldd, Pk, ldd, k, nt, k, 1, MODE_PIVOT_ROW, 0};
+      // C rows are the pivot rows themselves: ti0 == k so the local row offset is 0
+      int s2 = prof_begin(PK_FW_P2, st);
+      status = launch_tiles(J, nt - 1, st);
+      prof_end(s2, st, (nt - 1) * tile_ops);
+      if (status != EAR_OK) break;
+      cudaError_t e = cudaMemcpy2DAsync(prow, sizeof(int32_t) * Np, Pk, sizeof(int32_t) * ldd,
+                                        sizeof(int32_t) * Np, TILE, cudaMemcpyDeviceToDevice, st);
+      if (e != cudaSuccess) { set_error("pivot copy: %s", cudaGetErrorString(e)); status = EAR_ECUDA; break; }
+    }
+    int sc = prof_begin(PK_COMM, st);
+    status = comm_bcast(comm, prow, (int64_t)TILE * Np, owner, st);
+    prof_end(sc, st, 0);
+    if (status != EAR_OK) break;
+    dim3 g(16, nti);
+    EAR_LAUNCH(k_col_tiles_from_pivot, g, 256, 0, st)(Dblk, ldd, prow, Np, k, ti0, nti);
+    const int rows_here = (owner == rank) ? nti - 1 : nti;
+    TileJob J{Dblk, ldd, prow, Np, k, nt, ti0, nti, MODE_ROWS, 0};
+    int s3 = prof_begin(PK_FW_P3, st);
+    status = launch_tiles(J, (int64_t)rows_here * (nt - 1), st);
+    prof_end(s3, st, (double)rows_here * (nt - 1) * tile_ops);
+  }
+  cudaFreeAsync(prow, st);
+  if (status != EAR_OK) return status;
+  EAR_CUDA_TRY(cudaGetLastError());
+  return EAR_OK;
+}
+
+}  // namespace ear

@@ -1,0 +1,301 @@
+"""Thin ctypes binding of libearapsp.so (include/ear_apsp.h) -- argument marshalling only.
+
+Every step of the hot path runs in the library's CUDA kernels; torch is used only for device memory,
+streams and (for multi-GPU) the process group that distributes the NCCL unique id.  There is no CPU
+fallback: if the shared library is missing or cannot be loaded, every call raises.
+
+Names follow the C ABI (and the paper's Algorithm 1):
+    ear_decompose  -> Plan        Phase I, Reduce(G)
+    apsp_reduced(plan, D)         Phase II, APSP on G^r         (blocked FW)
+    expand_ears(plan, D, ...)     Phase III, UPDATE_DISTANCE
+    apsp_full(...)                all of Algorithm 1
+    apsp_full_host(...)           all of Algorithm 1 with host buffers (end-to-end)
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+from dataclasses import dataclass
+
+import numpy as np
+import torch
+
+from . import _build
+
+INF = 0x3FFFFFFF
+TILE = 128
+FLAG_NONE = 0
+FLAG_NO_CONTRACT = 1
+
+_lib = None
+
+
+class EarError(RuntimeError):
+    pass
+
+
+class _Info(ctypes.Structure):
+    _fields_ = [("n", ctypes.c_int32), ("n_reduced", ctypes.c_int32), ("n_reduced_padded", ctypes.c_int32),
+                ("n_chains", ctypes.c_int32), ("max_chain_len", ctypes.c_int32), ("n_promoted", ctypes.c_int32),
+                ("n_reduced_edges", ctypes.c_int64), ("m_simple", ctypes.c_int64), ("rank_rounds", ctypes.c_int32),
+                ("max_weight", ctypes.c_int32)]
+
+
+class _Profile(ctypes.Structure):
+    _fields_ = [("launches", ctypes.c_int64), ("decompose_ms", ctypes.c_double), ("fw_init_ms", ctypes.c_double),
+                ("fw_phase1_ms", ctypes.c_double), ("fw_phase2_ms", ctypes.c_double), ("fw_phase3_ms", ctypes.c_double),
+                ("fw_phase1_launches", ctypes.c_int64), ("fw_phase2_launches", ctypes.c_int64),
+                ("fw_phase3_launches", ctypes.c_int64), ("fw_phase2_minplus", ctypes.c_double),
+                ("fw_phase3_minplus", ctypes.c_double), ("comm_ms", ctypes.c_double), ("expand_ms", ctypes.c_double),
+                ("same_chain_ms", ctypes.c_double), ("expand_launches", ctypes.c_int64),
+                ("expand_bytes", ctypes.c_double)]
+
+
+# (name, restype, argtypes) for every symbol declared in include/ear_apsp.h
+_P, _I32, _I64, _U32 = ctypes.c_void_p, ctypes.c_int32, ctypes.c_int64, ctypes.c_uint32
+SIGNATURES = {
+    "ear_decompose": (_I32, [_I32, _I64, _P, _P, _P, _U32, _P, ctypes.POINTER(_P)]),
+    "ear_plan_info": (_I32, [_P, _I32, ctypes.POINTER(_Info)]),
+    "ear_plan_export": (_I32, [_P, _P, _P, _P, _P, _P, _P, _P]),
+    "ear_plan_export_reduced_edges": (_I32, [_P, _P, _P, _P, _P]),
+    "ear_plan_destroy": (None, [_P]),
+    "apsp_reduced": (_I32, [_P, _P, _I64, _P, _P]),
+    "ear_gather_reduced": (_I32, [_P, _P, _I64, _P, _I64, _P, _P]),
+    "expand_ears": (_I32, [_P, _P, _I64, _I32, _I32, _P, _I64, _P]),
+    "apsp_full": (_I32, [_I32, _I64, _P, _P, _P, _U32, _I32, _I32, _P, _I64, _P, _P]),
+    "apsp_full_host": (_I32, [_I32, _I64, _P, _P, _P, _U32, _I32, _I32, _P, _I64, _P, _P]),
+    "ear_row_block": (None, [_I32, _I32, _I32, ctypes.POINTER(_I32), ctypes.POINTER(_I32)]),
+    "ear_comm_unique_id": (_I32, [ctypes.c_char_p]),
+    "ear_comm_init": (_I32, [ctypes.c_char_p, _I32, _I32, ctypes.POINTER(_P)]),
+    "ear_comm_info": (_I32, [_P, ctypes.POINTER(_I32), ctypes.POINTER(_I32)]),
+    "ear_comm_destroy": (None, [_P]),
+    "ear_profile_enable": (None, [_I32]),
+    "ear_profile_reset": (None, []),
+    "ear_profile_read": (_I32, [ctypes.POINTER(_Profile)]),
+    "ear_status_string": (ctypes.c_char_p, [_I32]),
+    "ear_last_error": (ctypes.c_char_p, []),
+    "ear_version": (ctypes.c_char_p, []),
+}
+
+
+def lib_path() -> str:
+    return _build.LIB
+
+
+def lib():
+    """Load libearapsp.so (built in-tree by __graft_entry__.build()).  Raises if it is missing."""
+    global _lib
+    if _lib is None:
+        path = _build.LIB
+        if not os.path.exists(path):
+            raise EarError(f"{path} is missing: run __graft_entry__.build() (no CPU fallback exists)")
+        L = ctypes.CDLL(path)
+        for name, (res, args) in SIGNATURES.items():
+            f = getattr(L, name)
+            f.restype = res
+            f.argtypes = args
+        _lib = L
+    return _lib
+
+
+def _check(status: int, what: str):
+    if status != 0:
+        L = lib()
+        raise EarError(f"{what}: {L.ear_status_string(status).decode()} ({L.ear_last_error().decode()})")
+
+
+def _stream(stream=None) -> int:
+    if stream is None:
+        stream = torch.cuda.current_stream()
+    return stream.cuda_stream
+
+
+def _dev_i32(t: torch.Tensor, name: str) -> torch.Tensor:
+    if not (t.is_cuda and t.dtype == torch.int32 and t.is_contiguous()):
+        raise EarError(f"{name} must be a contiguous int32 CUDA tensor")
+    return t
+
+
+@dataclass
+class PlanInfo:
+    n: int
+    n_reduced: int
+    n_reduced_padded: int
+    n_chains: int
+    max_chain_len: int
+    n_promoted: int
+    n_reduced_edges: int
+    m_simple: int
+    rank_rounds: int
+    max_weight: int
+
+
+class Comm:
+    """NCCL communicator of this rank (one process per GPU), created collectively.  The unique id is
+    made on rank 0 by the library and distributed with torch.distributed."""
+
+    def __init__(self, handle, nranks: int, rank: int):
+        self.handle, self.nranks, self.rank = handle, nranks, rank
+
+    @classmethod
+    def from_torch_distributed(cls, group=None) -> "Comm":
+        import torch.distributed as dist
+        rank, world = dist.get_rank(group), dist.get_world_size(group)
+        buf = ctypes.create_string_buffer(128)
+        if rank == 0:
+            _check(lib().ear_comm_unique_id(buf), "ear_comm_unique_id")
+        obj = [bytes(buf.raw)]
+        dist.broadcast_object_list(obj, src=0, group=group)
+        h = _P()
+        _check(lib().ear_comm_init(obj[0], world, rank, ctypes.byref(h)), "ear_comm_init")
+        return cls(h, world, rank)
+
+    def destroy(self):
+        if self.handle:
+            lib().ear_comm_destroy(self.handle)
+            self.handle = None
+
+
+def _comm_handle(comm):
+    return None if comm is None else comm.handle
+
+
+class Plan:
+    """Reduce(G) result (library-owned device descriptors)."""
+
+    def __init__(self, handle, n):
+        self.handle, self.n = handle, n
+
+    def info(self, nranks: int = 1) -> PlanInfo:
+        i = _Info()
+        _check(lib().ear_plan_info(self.handle, nranks, ctypes.byref(i)), "ear_plan_info")
+        return PlanInfo(*[getattr(i, f) for f, _ in _Info._fields_])
+
+    def export(self, stream=None) -> dict:
+        """Per-vertex descriptors as CUDA int32 tensors (tests)."""
+        names = ["tid", "ear", "left", "right", "off_left", "off_right"]
+        out = {k: torch.empty(self.n, dtype=torch.int32, device="cuda") for k in names}
+        _check(lib().ear_plan_export(self.handle, *[out[k].data_ptr() for k in names], _stream(stream)),
+               "ear_plan_export")
+        return out
+
+    def reduced_edges(self, stream=None):
+        e = self.info().n_reduced_edges
+        u, v, w = (torch.empty(max(e, 1), dtype=torch.int32, device="cuda") for _ in range(3))
+        _check(lib().ear_plan_export_reduced_edges(self.handle, u.data_ptr(), v.data_ptr(), w.data_ptr(),
+                                                   _stream(stream)), "ear_plan_export_reduced_edges")
+        return u[:e], v[:e], w[:e]
+
+    def destroy(self):
+        if self.handle:
+            lib().ear_plan_destroy(self.handle)
+            self.handle = None
+
+    def __del__(self):  # pragma: no cover
+        try:
+            self.destroy()
+        except Exception:
+            pass
+
+
+def ear_decompose(n: int, src: torch.Tensor, dst: torch.Tensor, w: torch.Tensor, flags: int = 0,
+                  stream=None) -> Plan:
+    src, dst, w = _dev_i32(src, "src"), _dev_i32(dst, "dst"), _dev_i32(w, "w")
+    h = _P()
+    _check(lib().ear_decompose(n, src.numel(), src.data_ptr(), dst.data_ptr(), w.data_ptr(), flags,
+                               _stream(stream), ctypes.byref(h)), "ear_decompose")
+    return Plan(h, n)
+
+
+def alloc_D(plan: Plan, comm: Comm | None = None) -> torch.Tensor:
+    """Device buffer for apsp_reduced: full Np x Np (single GPU) or this rank's (Np/P) x Np block."""
+    P = 1 if comm is None else comm.nranks
+    Np = plan.info(P).n_reduced_padded
+    return torch.empty((Np // P, Np), dtype=torch.int32, device="cuda")
+
+
+def apsp_reduced(plan: Plan, D: torch.Tensor, comm: Comm | None = None, stream=None) -> torch.Tensor:
+    D = _dev_i32(D, "D")
+    _check(lib().apsp_reduced(plan.handle, D.data_ptr(), D.stride(0), _comm_handle(comm), _stream(stream)),
+           "apsp_reduced")
+    return D
+
+
+def gather_reduced(plan: Plan, D_block: torch.Tensor, comm: Comm, D_full: torch.Tensor | None = None,
+                   stream=None) -> torch.Tensor:
+    Np = plan.info(comm.nranks).n_reduced_padded
+    if D_full is None:
+        D_full = torch.empty((Np, Np), dtype=torch.int32, device="cuda")
+    _check(lib().ear_gather_reduced(plan.handle, D_block.data_ptr(), D_block.stride(0), D_full.data_ptr(),
+                                    D_full.stride(0), _comm_handle(comm), _stream(stream)), "ear_gather_reduced")
+    return D_full
+
+
+def expand_ears(plan: Plan, D_full: torch.Tensor, row_begin: int, row_end: int, out: torch.Tensor | None = None,
+                stream=None) -> torch.Tensor:
+    if out is None:
+        out = torch.empty((row_end - row_begin, plan.n), dtype=torch.int32, device="cuda")
+    _dev_i32(D_full, "D_full")
+    if not (out.is_cuda and out.dtype == torch.int32 and out.stride(1) == 1):
+        raise EarError("out must be an int32 CUDA tensor with unit column stride")
+    _check(lib().expand_ears(plan.handle, D_full.data_ptr(), D_full.stride(0), row_begin, row_end, out.data_ptr(),
+                             out.stride(0), _stream(stream)), "expand_ears")
+    return out
+
+
+def row_block(rows: int, nranks: int, rank: int):
+    b, e = _I32(), _I32()
+    lib().ear_row_block(rows, nranks, rank, ctypes.byref(b), ctypes.byref(e))
+    return b.value, e.value
+
+
+def apsp_full(n: int, src: torch.Tensor, dst: torch.Tensor, w: torch.Tensor, out: torch.Tensor | None = None,
+              row_begin: int = 0, row_end: int | None = None, flags: int = 0, comm: Comm | None = None,
+              stream=None) -> torch.Tensor:
+    """Algorithm 1 APSP(G) on device buffers: rows [row_begin, row_end) of S (caller order)."""
+    row_end = n if row_end is None else row_end
+    src, dst, w = _dev_i32(src, "src"), _dev_i32(dst, "dst"), _dev_i32(w, "w")
+    if out is None:
+        out = torch.empty((row_end - row_begin, n), dtype=torch.int32, device="cuda")
+    _check(lib().apsp_full(n, src.numel(), src.data_ptr(), dst.data_ptr(), w.data_ptr(), flags, row_begin, row_end,
+                           out.data_ptr(), out.stride(0), _comm_handle(comm), _stream(stream)), "apsp_full")
+    return out
+
+
+def apsp_full_host(n: int, src: np.ndarray | torch.Tensor, dst, w, out: torch.Tensor | None = None,
+                   row_begin: int = 0, row_end: int | None = None, flags: int = 0, comm: Comm | None = None,
+                   stream=None) -> torch.Tensor:
+    """Algorithm 1 APSP(G) from HOST edge arrays into a HOST (preferably pinned) int32 tensor."""
+    row_end = n if row_end is None else row_end
+    tens = [torch.as_tensor(np.ascontiguousarray(x, dtype=np.int32)) if not isinstance(x, torch.Tensor) else x
+            for x in (src, dst, w)]
+    for t in tens:
+        if t.is_cuda or t.dtype != torch.int32 or not t.is_contiguous():
+            raise EarError("apsp_full_host takes contiguous int32 host arrays")
+    if out is None:
+        out = torch.empty((row_end - row_begin, n), dtype=torch.int32, pin_memory=True)
+    if out.is_cuda or out.dtype != torch.int32 or out.stride(1) != 1:
+        raise EarError("out must be a host int32 tensor with unit column stride")
+    _check(lib().apsp_full_host(n, tens[0].numel(), tens[0].data_ptr(), tens[1].data_ptr(), tens[2].data_ptr(),
+                                flags, row_begin, row_end, out.data_ptr(), out.stride(0), _comm_handle(comm),
+                                _stream(stream)), "apsp_full_host")
+    return out
+
+
+def profile_enable(on: bool = True):
+    """CUDA-event timing of every library kernel launch (per kernel class), see ear_profile_t."""
+    lib().ear_profile_enable(1 if on else 0)
+
+
+def profile_reset():
+    lib().ear_profile_reset()
+
+
+def profile_read() -> dict:
+    p = _Profile()
+    _check(lib().ear_profile_read(ctypes.byref(p)), "ear_profile_read")
+    return {f: getattr(p, f) for f, _ in _Profile._fields_}
+
+
+def version() -> str:
+    return lib().ear_version().decode()
