@@ -1,0 +1,388 @@
+#!/usr/bin/env python
+"""Benchmark: full APSP distance entries/s of the ear-reduced B200 path (BASELINE.json metric).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config cfg4] [--impl ours|reference]
+
+One step = one pass of the whole hot path over the workload: apsp_full =
+Reduce(G) chain contraction -> blocked min-plus FW on G^r -> ear expansion of this rank's rows of the
+N x N int32 matrix, graph already resident in HBM.  For N > 1 GPUs (torchrun, one process per GPU)
+the FW is row-block sharded with a per-round NCCL pivot broadcast and every rank expands its own row
+block; the total work is fixed (strong scaling).  Timing: W untimed warm-up steps, then exactly K
+steps between barrier + synchronize, CUDA events on the launching stream, max over ranks.  D (3.6 GB)
+and the output (40 GB) are far larger than L2, so no flush is needed between steps.
+
+Rank 0 prints one JSON line.  Extra keys: roofline (dominant kernel = FW phase-3 min-plus tile
+kernel, ALU bound), roofline_expand (HBM bound), cpu_baseline (the CPU oracle on a bounded sample,
+rank 0 at N = 1 only), e2e (the same metric through the host-buffer C-ABI call apsp_full_host with
+every step's H2D edge upload and D2H copy of the output rows), clocks, gpu_launches, phases_ms.
+
+--impl reference runs the CPU oracle (Dijkstra from every source of a bounded sample of sources on
+all host cores) as the reference arm; under torchrun only rank 0 runs it.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+if ROOT not in sys.path:
+    sys.path.insert(0, ROOT)
+
+METRIC = "full APSP distance entries/sec at 1/2/4/8 B200; min-plus GOPS & HBM GB/s"
+UNIT = "entries/s"
+SM_COUNT = 148
+ALU_LANES_PER_SM = 64          # VIADDMNMX issue rate measured by microbench/minplus_peak.cu
+WORKLOADS = {
+    "cfg1": "cfg1: 33x33 torus + 911 degree-two subdivisions (N=2,000, 45.6% degree two)",
+    "cfg2": "cfg2: 89x89 open grid subdivided to N=20,000 (road-like, 60% degree two)",
+    "cfg3_f0": "cfg3 f=0%: 200x250 torus, N=50,000 (no degree-two vertices)",
+    "cfg3_f20": "cfg3 f=20%: 200x200 torus + 10,000 subdivisions, N=50,000",
+    "cfg3_f40": "cfg3 f=40%: 150x200 torus + 20,000 subdivisions, N=50,000",
+    "cfg3_f60": "cfg3 f=60%: 100x200 torus + 30,000 subdivisions, N=50,000",
+    "cfg3_f80": "cfg3 f=80%: 100x100 torus + 40,000 subdivisions, N=50,000",
+    "cfg4": "cfg4: power-grid-like (28,500-point 3-NN geometric graph + 5% pendants, chained components, "
+            "degree-two subdivisions), N=100,000, ~30k reduced vertices, 40 GB int32 distance matrix",
+    "cfg5": "cfg5: power-grid-like, N=200,000, ~60k reduced vertices, 160 GB int32 distance matrix",
+}
+
+
+def log(*a):
+    print(*a, file=sys.stderr, flush=True)
+
+
+def max_over_ranks(x: float, world: int, device) -> float:
+    """Max of a per-rank time over all ranks (the contract's multi-GPU timing rule)."""
+    if world == 1:
+        return x
+    import torch
+    import torch.distributed as dist
+    t = torch.tensor([x], dtype=torch.float64, device=device)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return float(t.item())
+
+
+# ------------------------------------------------------------------------------------ clocks
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled every 200 ms during the timed region."""
+
+    FIELDS = ["clocks.sm", "clocks.max.sm", "power.draw", "clocks_event_reasons.hw_slowdown",
+              "clocks_event_reasons.hw_thermal_slowdown", "clocks_event_reasons.sw_thermal_slowdown",
+              "clocks_event_reasons.sw_power_cap"]
+
+    def __init__(self, gpu_id: str):
+        self.gpu_id, self.lines, self.proc = gpu_id, [], None
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", self.gpu_id, "--query-gpu=" + ",".join(self.FIELDS),
+                                          "--format=csv,noheader,nounits", "-lms", "200"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception as e:  # pragma: no cover
+            log("clock sampler unavailable:", e)
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def stop(self) -> dict:
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": [], "samples": 0}
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        self.t.join(timeout=2)
+        sm, mx, pw, reasons = [], [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            p = [x.strip() for x in ln.split(",")]
+            if len(p) != len(self.FIELDS):
+                continue
+            try:
+                sm.append(float(p[0])); mx.append(float(p[1])); pw.append(float(p[2]))
+            except ValueError:
+                continue
+            for nm, v in zip(names, p[3:]):
+                if v.lower().startswith("active"):
+                    reasons.add(nm)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "power_w_max": max(pw) if pw else None, "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def gpu_id_for(dev_index: int) -> str:
+    import torch
+    try:
+        u = str(torch.cuda.get_device_properties(dev_index).uuid)
+        return u if u.startswith("GPU-") else "GPU-" + u
+    except Exception:
+        vis = os.environ.get("CUDA_VISIBLE_DEVICES")
+        return vis.split(",")[dev_index] if vis else str(dev_index)
+
+
+def measured_peaks() -> dict:
+    try:
+        return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
+    except Exception:
+        return {}
+
+
+def ncu_traffic(kernel_key: str, workload: str):
+    """Per-launch DRAM bytes of a kernel from the committed ncu --set full summary (or None)."""
+    path = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    try:
+        d = json.load(open(path))
+        e = d.get(workload, {}).get(kernel_key)
+        return None if e is None else float(e["dram_bytes_per_launch"])
+    except Exception:
+        return None
+
+
+# ------------------------------------------------------------------------------------ CPU oracle
+def oracle_sample(g, target_s: float, rows_hint: int | None = None):
+    """Time the CPU oracle (as it stands) on a bounded sample of source rows: returns
+    (entries_per_s, rows, seconds, threads)."""
+    import numpy as np
+
+    import oracle
+    threads = oracle.num_threads()
+    if rows_hint is None:
+        probe = min(g.n, max(threads * 2, 32))
+        t = time.perf_counter()
+        oracle.apsp_rows(g.n, g.src, g.dst, g.w, np.arange(probe))
+        dt = time.perf_counter() - t
+        rows_hint = int(min(g.n, max(probe, probe * target_s / max(dt, 1e-6))))
+    rows = np.arange(rows_hint) % g.n
+    t = time.perf_counter()
+    oracle.apsp_rows(g.n, g.src, g.dst, g.w, rows)
+    dt = time.perf_counter() - t
+    return rows_hint * g.n / dt, rows_hint, dt, threads
+
+
+def run_reference(args, rank, world):
+    """The reference arm for this tier: the CPU oracle, timed on the box's host cores."""
+    if rank != 0:
+        return
+    import numpy as np
+
+    import oracle
+    from paper_conf_ipps_duttackb17_b200 import graphgen as gg
+    g = gg.config(args.config, args.seed)
+    threads = oracle.num_threads()
+    # size one step to ~2-3 s of all-core CPU work
+    probe = max(threads * 2, 32)
+    t = time.perf_counter()
+    oracle.apsp_rows(g.n, g.src, g.dst, g.w, np.arange(probe))
+    per_row = (time.perf_counter() - t) / probe
+    rows_per_step = int(min(g.n, max(threads, 2.5 / max(per_row, 1e-9))))
+    for i in range(args.warmup):
+        oracle.apsp_rows(g.n, g.src, g.dst, g.w, (np.arange(rows_per_step) + i * rows_per_step) % g.n)
+    t = time.perf_counter()
+    for i in range(args.steps):
+        oracle.apsp_rows(g.n, g.src, g.dst, g.w, (np.arange(rows_per_step) + i * rows_per_step) % g.n)
+    dt = time.perf_counter() - t
+    value = rows_per_step * g.n * args.steps / dt
+    sample = (f"{rows_per_step} Dijkstra sources per step on the uncontracted {args.config} graph "
+              f"(N={g.n}); entries = sources x N")
+    line = {"metric": METRIC, "value": value, "unit": UNIT, "impl": "reference", "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": dt / args.steps * 1e3,
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "int64 (int32 output)",
+            "data": "synthetic (seeded generator)",
+            "config": {"workload": WORKLOADS.get(args.config, args.config), "name": args.config, "n": g.n,
+                       "m": g.m, "seed": args.seed},
+            "cpu_baseline": {"value": value, "unit": UNIT, "cores": threads, "kind": "oracle", "sample": sample},
+            "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+# ------------------------------------------------------------------------------------ our arm
+def run_ours(args, rank, world, local_rank):
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_ipps_duttackb17_b200 as ea
+    from paper_conf_ipps_duttackb17_b200 import graphgen as gg
+
+    torch.cuda.set_device(local_rank)
+    dev = torch.device("cuda", local_rank)
+    comm = None
+    if world > 1:
+        comm = ea.Comm.from_torch_distributed()
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+
+    t0 = time.perf_counter()
+    g = gg.config(args.config, args.seed)
+    stats = gg.stats(g)
+    log(f"[rank {rank}] generated {args.config}: n={g.n} m={g.m} in {time.perf_counter() - t0:.1f}s")
+    src = torch.as_tensor(g.src).to(dev)
+    dst = torch.as_tensor(g.dst).to(dev)
+    w = torch.as_tensor(g.w).to(dev)
+    r0, r1 = ea.row_block(g.n, world, rank)
+    rows = r1 - r0
+    out = torch.empty((rows, g.n), dtype=torch.int32, device=dev)
+    plan = ea.ear_decompose(g.n, src, dst, w)
+    info = plan.info(world)
+    plan.destroy()
+    stream = torch.cuda.current_stream(dev)
+
+    def step():
+        ea.apsp_full(g.n, src, dst, w, out=out, row_begin=r0, row_end=r1, comm=comm, stream=stream)
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    barrier()
+    torch.cuda.synchronize()
+
+    sampler = ClockSampler(gpu_id_for(local_rank))
+    sampler.start()
+    time.sleep(0.3)
+    ea.profile_reset()
+    ea.profile_enable(True)
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    ev0.record(stream)
+    for _ in range(args.steps):
+        step()
+    ev1.record(stream)
+    torch.cuda.synchronize()
+    barrier()
+    torch.cuda.synchronize()
+    clocks = sampler.stop()
+    prof = ea.profile_read()
+    ea.profile_enable(False)
+    ms = ev0.elapsed_time(ev1)
+    ms_max = max_over_ranks(ms, world, dev)
+    value = float(g.n) * float(g.n) * args.steps / (ms_max / 1e3)
+
+    # roofline of the dominant kernel: FW phase-3 min-plus tiles (ALU bound)
+    peaks = measured_peaks()
+    sm_max = float(peaks.get("sm_max_mhz", 1965.0))
+    peak_alu = SM_COUNT * ALU_LANES_PER_SM * sm_max * 1e6 / 1e12     # T min-plus / s
+    p3_ms = prof["fw_phase3_ms"]
+    ach = prof["fw_phase3_minplus"] / (p3_ms / 1e3) / 1e12 if p3_ms > 0 else 0.0
+    n_p3 = max(prof["fw_phase3_launches"], 1)
+    roofline = {"bound": "alu", "kernel": "k_fw_tiles (FW phase 3)", "achieved": ach, "peak": peak_alu,
+                "unit": "Tminplus/s", "frac": ach / peak_alu if peak_alu else None,
+                "traffic": ncu_traffic("k_fw_tiles", args.config),
+                "avg_launch_ms": p3_ms / n_p3, "minplus_per_launch": prof["fw_phase3_minplus"] / n_p3,
+                "peak_basis": f"{SM_COUNT} SMs x {ALU_LANES_PER_SM} VIADDMNMX/clk/SM x {sm_max:.0f} MHz "
+                              "(sm_max_mhz of MEASURED_PEAKS.json; issue rate from microbench/minplus_peak.cu)"}
+    if clocks.get("sm_mhz"):
+        roofline["frac_at_run_clock"] = ach / (SM_COUNT * ALU_LANES_PER_SM * clocks["sm_mhz"] * 1e6 / 1e12)
+    hbm = float(peaks.get("hbm_gbs", 6555.2))
+    ex_ms = prof["expand_ms"]
+    ex_ach = prof["expand_bytes"] / (ex_ms / 1e3) / 1e9 if ex_ms > 0 else 0.0
+    roofline_expand = {"bound": "hbm", "kernel": "k_expand", "achieved": ex_ach, "peak": hbm, "unit": "GB/s",
+                       "frac": ex_ach / hbm, "traffic": ncu_traffic("k_expand", args.config),
+                       "avg_launch_ms": ex_ms / max(prof["expand_launches"], 1),
+                       "bytes_per_launch": prof["expand_bytes"] / max(prof["expand_launches"], 1)}
+    K = args.steps
+    fw_ms = prof["fw_init_ms"] + prof["fw_phase1_ms"] + prof["fw_phase2_ms"] + prof["fw_phase3_ms"]
+    phases = {"decompose": prof["decompose_ms"] / K, "fw": fw_ms / K, "fw_phase1": prof["fw_phase1_ms"] / K,
+              "fw_phase2": prof["fw_phase2_ms"] / K, "fw_phase3": p3_ms / K, "comm": prof["comm_ms"] / K,
+              "expand": ex_ms / K, "same_chain": prof["same_chain_ms"] / K}
+    fw_minplus = prof["fw_phase2_minplus"] + prof["fw_phase3_minplus"]
+    del out
+    torch.cuda.empty_cache()
+
+    # e2e through the host-buffer C-ABI entry point: H2D edges + D2H output rows inside the region
+    e2e = None
+    if not args.no_e2e:
+        hs = torch.as_tensor(g.src).pin_memory()
+        hd = torch.as_tensor(g.dst).pin_memory()
+        hw = torch.as_tensor(g.w).pin_memory()
+        hout = torch.empty((rows, g.n), dtype=torch.int32, pin_memory=True)
+        e2e_steps = max(1, min(args.steps, args.e2e_steps))
+        ea.apsp_full_host(g.n, hs, hd, hw, out=hout, row_begin=r0, row_end=r1, comm=comm, stream=stream)
+        barrier()
+        t = time.perf_counter()
+        for _ in range(e2e_steps):
+            ea.apsp_full_host(g.n, hs, hd, hw, out=hout, row_begin=r0, row_end=r1, comm=comm, stream=stream)
+        torch.cuda.synchronize()
+        e2e_s = max_over_ranks(time.perf_counter() - t, world, dev)
+        barrier()
+        e2e = {"value": float(g.n) * g.n * e2e_steps / e2e_s, "unit": UNIT, "h2d_bytes_per_step": 3 * 4 * g.m,
+               "d2h_bytes_per_step": 4 * rows * g.n, "steps": e2e_steps,
+               "api": "apsp_full_host (pinned host edge list in, pinned host rows out)"}
+        del hout
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        v, nrows, dt, thr = oracle_sample(g, args.cpu_seconds)
+        cpu = {"value": v, "unit": UNIT, "cores": thr, "kind": "oracle",
+               "sample": f"Dijkstra from the first {nrows} sources of the uncontracted {args.config} graph "
+                         f"({dt:.1f} s on {thr} threads); entries = sources x N"}
+
+    launches = int(prof["launches"])
+    if rank == 0:
+        line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": K, "warmup": args.warmup,
+                "ms_per_step": ms_max / K, "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
+                "dtype": "int32", "data": "synthetic (seeded generator, spatially coherent labels)",
+                "config": {"workload": WORKLOADS.get(args.config, args.config), "name": args.config,
+                           "n": g.n, "m": g.m, "n_reduced": info.n_reduced, "n_reduced_padded": info.n_reduced_padded,
+                           "n_chains": info.n_chains, "max_chain_len": info.max_chain_len,
+                           "degree2_frac": stats["deg2_frac"], "seed": args.seed, "rows_per_rank": rows,
+                           "parallelism": f"row-block x{world}" if world > 1 else "single GPU",
+                           "l2": "inputs larger than L2 (D %.1f GB, output %.1f GB per step)" % (
+                               4.0 * info.n_reduced_padded ** 2 / 1e9, 4.0 * g.n * g.n / 1e9)},
+                "roofline": roofline, "roofline_expand": roofline_expand,
+                "fw_minplus_gops": fw_minplus / (fw_ms / 1e3) / 1e9 if fw_ms > 0 else None,
+                "phases_ms": phases, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks,
+                "gpu_launches": launches,
+                "gpu_launches_note": "own kernels in the timed region (CUB sort/scan launches of Phase I excluded)",
+                "mteps_context": g.m * g.n / (ms_max / K / 1e3) / 1e6}
+        print(json.dumps(line), flush=True)
+    if comm is not None:
+        comm.destroy()
+
+
+def main():
+    ap = argparse.ArgumentParser(description=__doc__, formatter_class=argparse.RawDescriptionHelpFormatter)
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", default="cfg4")
+    ap.add_argument("--seed", type=int, default=0)
+    ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--e2e-steps", type=int, default=2)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-seconds", type=float, default=15.0)
+    args = ap.parse_args()
+
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    if world != args.gpus:
+        log(f"note: --gpus {args.gpus} but WORLD_SIZE={world}; using WORLD_SIZE")
+    if args.impl == "reference":
+        run_reference(args, rank, world)
+        return
+    if world > 1:
+        import torch
+        import torch.distributed as dist
+        torch.cuda.set_device(local_rank)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+    try:
+        run_ours(args, rank, world, local_rank)
+    finally:
+        if world > 1:
+            import torch.distributed as dist
+            dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

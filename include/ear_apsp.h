@@ -113,6 +113,14 @@ void ear_plan_destroy(ear_plan_t plan);
  * Asynchronous.  Errors: EAR_EINVAL (ldd too small/misaligned), EAR_ENCCL, EAR_ECUDA. */
 ear_status_t apsp_reduced(ear_plan_t plan, int32_t *d_D, int64_t ldd, ear_comm_t comm, void *stream);
 
+/* The row-block-sharded schedule of apsp_reduced for `nranks` ranks, emulated in ONE process on the
+ * current device: the same per-rank kernels and addressing, rank r's rows at d_D + r*(Np/P)*ldd, and
+ * the pivot broadcast replaced by the shared pivot-row buffer.  d_D is the full Np x Np matrix
+ * (Np = ear_plan_info(nranks).n_reduced_padded).  Used to test the multi-GPU path on one GPU; the
+ * result must equal apsp_reduced bit for bit.  Asynchronous; errors as apsp_reduced. */
+ear_status_t apsp_reduced_emulated(ear_plan_t plan, int32_t nranks, int32_t *d_D, int64_t ldd,
+                                   void *stream);
+
 /* All-gather the row blocks produced by apsp_reduced with `comm` into the full Np x Np matrix
  * d_D_full (ldd_full >= Np).  d_D_block may alias this rank's rows of d_D_full when
  * ldd_block == ldd_full and d_D_block == d_D_full + rank*(Np/P)*ldd_full. */

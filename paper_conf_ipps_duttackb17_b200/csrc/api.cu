@@ -152,6 +152,19 @@ ear_status_t apsp_reduced(ear_plan_t p, int32_t *d_D, int64_t ldd, ear_comm_t co
   return fw_sharded(d_D, ldd, Np, comm, st);
 }
 
+ear_status_t apsp_reduced_emulated(ear_plan_t p, int32_t nranks, int32_t *d_D, int64_t ldd, void *stream) {
+  g_err[0] = 0;
+  if (!p || !d_D || nranks < 1) { set_error("apsp_reduced_emulated: bad argument"); return EAR_EINVAL; }
+  const int32_t Np = padded(p, nranks);
+  if (ldd < Np || ldd % 4 != 0 || !aligned16(d_D)) {
+    set_error("apsp_reduced_emulated: need ldd >= Np=%d, ldd %% 4 == 0, 16-byte aligned D", Np);
+    return EAR_EINVAL;
+  }
+  cudaStream_t st = (cudaStream_t)stream;
+  EAR_TRY(fw_init_D(p, d_D, ldd, Np, 0, Np, st));
+  return fw_sharded_emulated(d_D, ldd, Np, nranks, st);
+}
+
 ear_status_t ear_gather_reduced(ear_plan_t p, const int32_t *d_D_block, int64_t ldd_block, int32_t *d_D_full,
                                 int64_t ldd_full, ear_comm_t comm, void *stream) {
   if (!p || !d_D_block || !d_D_full) { set_error("ear_gather_reduced: NULL argument"); return EAR_EINVAL; }

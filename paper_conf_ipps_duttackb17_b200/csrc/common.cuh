@@ -91,6 +91,7 @@ ear_status_t fw_init_D(const ear_plan_s *plan, int32_t *D, int64_t ldd, int32_t 
                        int32_t rows, cudaStream_t stream);
 ear_status_t fw_single(int32_t *D, int64_t ldd, int32_t Np, cudaStream_t stream);
 ear_status_t fw_sharded(int32_t *Dblk, int64_t ldd, int32_t Np, ear_comm_s *comm, cudaStream_t stream);
+ear_status_t fw_sharded_emulated(int32_t *D, int64_t ldd, int32_t Np, int32_t P, cudaStream_t stream);
 // expand.cu
 ear_status_t expand(const ear_plan_s *plan, const int32_t *D, int64_t ldd, int32_t row_begin,
                     int32_t row_end, int32_t *out, int64_t ldo, cudaStream_t stream);

@@ -312,46 +312,89 @@ ear_status_t fw_single(int32_t *D, int64_t ldd, int32_t Np, cudaStream_t st) {
   return EAR_OK;
 }
 
-// Row-block sharded: this rank holds rows [rank*R, (rank+1)*R) of D (R = Np / nranks, a multiple
-// of 128) in Dblk (leading dimension ldd).  Each round the owner of pivot block k closes the pivot
-// tile and its pivot-row tiles, the 128 x Np pivot row block is broadcast (NCCL), every rank fills
-// its column tiles by symmetry and updates its remaining tiles.
-ear_status_t fw_sharded(int32_t *Dblk, int64_t ldd, int32_t Np, ear_comm_s *comm, cudaStream_t st) {
-  const int nt = Np / TILE;
-  const int P = comm->nranks, rank = comm->rank;
-  const int nti = nt / P, ti0 = rank * nti;
+// Row-block sharded FW.  Rank r holds rows [r*R, (r+1)*R) of D (R = Np / P, a multiple of 128).
+// Round k: the owner of pivot block k closes the pivot tile and its pivot-row tiles and copies the
+// 128 x Np pivot row block into `prow`; the block reaches every rank (NCCL broadcast, or the same
+// buffer when emulated); every rank fills its pivot-column tiles by symmetry and updates its other
+// tiles with both operands taken from `prow`.
+struct ShardCtx {
+  int32_t *Dblk;    // this rank's row block
+  int64_t ldd;
+  int32_t Np, nt, P, rank, nti, ti0;
+  int32_t *prow;    // 128 x Np pivot row block (leading dimension Np)
+};
+
+static ShardCtx shard_ctx(int32_t *Dblk, int64_t ldd, int32_t Np, int32_t P, int32_t rank, int32_t *prow) {
+  ShardCtx c;
+  c.Dblk = Dblk; c.ldd = ldd; c.Np = Np; c.nt = Np / TILE; c.P = P; c.rank = rank;
+  c.nti = c.nt / P; c.ti0 = rank * c.nti; c.prow = prow;
+  return c;
+}
+
+static ear_status_t shard_owner_step(const ShardCtx &c, int k, cudaStream_t st) {
   const double tile_ops = (double)TILE * TILE * TILE;
+  int32_t *Pk = c.Dblk + (int64_t)(k - c.ti0) * TILE * c.ldd;
+  int s1 = prof_begin(PK_FW_P1, st);
+  EAR_LAUNCH(k_fw_phase1, 1, NT, 0, st)(Pk + (int64_t)k * TILE, c.ldd);
+  prof_end(s1, st, tile_ops);
+  // pivot-row tiles; C rows are the pivot rows themselves (ti0 = k: local row offset 0)
+  TileJob J{Pk, c.ldd, Pk, c.ldd, k, c.nt, k, 1, MODE_PIVOT_ROW, 0};
+  int s2 = prof_begin(PK_FW_P2, st);
+  EAR_TRY(launch_tiles(J, c.nt - 1, st));
+  prof_end(s2, st, (c.nt - 1) * tile_ops);
+  EAR_CUDA_TRY(cudaMemcpy2DAsync(c.prow, sizeof(int32_t) * c.Np, Pk, sizeof(int32_t) * c.ldd,
+                                 sizeof(int32_t) * c.Np, TILE, cudaMemcpyDeviceToDevice, st));
+  return EAR_OK;
+}
+
+static ear_status_t shard_update_step(const ShardCtx &c, int k, cudaStream_t st) {
+  const double tile_ops = (double)TILE * TILE * TILE;
+  const int owner = k / c.nti;
+  dim3 g(16, c.nti);
+  EAR_LAUNCH(k_col_tiles_from_pivot, g, 256, 0, st)(c.Dblk, c.ldd, c.prow, c.Np, k, c.ti0, c.nti);
+  const int rows_here = (owner == c.rank) ? c.nti - 1 : c.nti;
+  TileJob J{c.Dblk, c.ldd, c.prow, c.Np, k, c.nt, c.ti0, c.nti, MODE_ROWS, 0};
+  int s3 = prof_begin(PK_FW_P3, st);
+  EAR_TRY(launch_tiles(J, (int64_t)rows_here * (c.nt - 1), st));
+  prof_end(s3, st, (double)rows_here * (c.nt - 1) * tile_ops);
+  return EAR_OK;
+}
+
+ear_status_t fw_sharded(int32_t *Dblk, int64_t ldd, int32_t Np, ear_comm_s *comm, cudaStream_t st) {
   int32_t *prow = nullptr;
   EAR_CUDA_TRY(cudaMallocAsync((void **)&prow, sizeof(int32_t) * (size_t)TILE * Np, st));
+  const ShardCtx c = shard_ctx(Dblk, ldd, Np, comm->nranks, comm->rank, prow);
   ear_status_t status = EAR_OK;
-  for (int k = 0; k < nt && status == EAR_OK; ++k) {
-    const int owner = k / nti;
-    if (owner == rank) {
-      int32_t *Pk = Dblk + (int64_t)(k - ti0) * TILE * ldd;
-      int s1 = prof_begin(PK_FW_P1, st);
-      EAR_LAUNCH(k_fw_phase1, 1, NT, 0, st)(Pk + (int64_t)k * TILE, ldd);
-      prof_end(s1, st, tile_ops);
-      TileJob J{Pk, ldd, Pk, ldd, k, nt, k, 1, MODE_PIVOT_ROW, 0};
-      // C rows are the pivot rows themselves: ti0 == k so the local row offset is 0
-      int s2 = prof_begin(PK_FW_P2, st);
-      status = launch_tiles(J, nt - 1, st);
-      prof_end(s2, st, (nt - 1) * tile_ops);
-      if (status != EAR_OK) break;
-      cudaError_t e = cudaMemcpy2DAsync(prow, sizeof(int32_t) * Np, Pk, sizeof(int32_t) * ldd,
-                                        sizeof(int32_t) * Np, TILE, cudaMemcpyDeviceToDevice, st);
-      if (e != cudaSuccess) { set_error("pivot copy: %s", cudaGetErrorString(e)); status = EAR_ECUDA; break; }
-    }
+  for (int k = 0; k < c.nt && status == EAR_OK; ++k) {
+    const int owner = k / c.nti;
+    if (owner == c.rank) status = shard_owner_step(c, k, st);
+    if (status != EAR_OK) break;
     int sc = prof_begin(PK_COMM, st);
     status = comm_bcast(comm, prow, (int64_t)TILE * Np, owner, st);
     prof_end(sc, st, 0);
     if (status != EAR_OK) break;
-    dim3 g(16, nti);
-    EAR_LAUNCH(k_col_tiles_from_pivot, g, 256, 0, st)(Dblk, ldd, prow, Np, k, ti0, nti);
-    const int rows_here = (owner == rank) ? nti - 1 : nti;
-    TileJob J{Dblk, ldd, prow, Np, k, nt, ti0, nti, MODE_ROWS, 0};
-    int s3 = prof_begin(PK_FW_P3, st);
-    status = launch_tiles(J, (int64_t)rows_here * (nt - 1), st);
-    prof_end(s3, st, (double)rows_here * (nt - 1) * tile_ops);
+    status = shard_update_step(c, k, st);
+  }
+  cudaFreeAsync(prow, st);
+  if (status != EAR_OK) return status;
+  EAR_CUDA_TRY(cudaGetLastError());
+  return EAR_OK;
+}
+
+// The same schedule for P ranks emulated in one process on one device (tests of the multi-GPU
+// path on a single GPU): D is the full matrix, rank r's block starts at row r*Np/P, and the
+// broadcast is the shared pivot-row buffer itself.
+ear_status_t fw_sharded_emulated(int32_t *D, int64_t ldd, int32_t Np, int32_t P, cudaStream_t st) {
+  int32_t *prow = nullptr;
+  EAR_CUDA_TRY(cudaMallocAsync((void **)&prow, sizeof(int32_t) * (size_t)TILE * Np, st));
+  const int32_t R = Np / P;
+  ear_status_t status = EAR_OK;
+  const int nt = Np / TILE, nti = nt / P;
+  for (int k = 0; k < nt && status == EAR_OK; ++k) {
+    const int owner = k / nti;
+    status = shard_owner_step(shard_ctx(D + (int64_t)owner * R * ldd, ldd, Np, P, owner, prow), k, st);
+    for (int r = 0; r < P && status == EAR_OK; ++r)
+      status = shard_update_step(shard_ctx(D + (int64_t)r * R * ldd, ldd, Np, P, r, prow), k, st);
   }
   cudaFreeAsync(prow, st);
   if (status != EAR_OK) return status;

@@ -60,6 +60,7 @@ SIGNATURES = {
     "ear_plan_export_reduced_edges": (_I32, [_P, _P, _P, _P, _P]),
     "ear_plan_destroy": (None, [_P]),
     "apsp_reduced": (_I32, [_P, _P, _I64, _P, _P]),
+    "apsp_reduced_emulated": (_I32, [_P, _I32, _P, _I64, _P]),
     "ear_gather_reduced": (_I32, [_P, _P, _I64, _P, _I64, _P, _P]),
     "expand_ears": (_I32, [_P, _P, _I64, _I32, _I32, _P, _I64, _P]),
     "apsp_full": (_I32, [_I32, _I64, _P, _P, _P, _U32, _I32, _I32, _P, _I64, _P, _P]),
@@ -137,17 +138,24 @@ class Comm:
     def __init__(self, handle, nranks: int, rank: int):
         self.handle, self.nranks, self.rank = handle, nranks, rank
 
+    @staticmethod
+    def distribute_unique_id(group=None) -> bytes:
+        """Rank 0 creates the NCCL unique id (library call); torch.distributed broadcasts it."""
+        import torch.distributed as dist
+        buf = ctypes.create_string_buffer(128)
+        if dist.get_rank(group) == 0:
+            _check(lib().ear_comm_unique_id(buf), "ear_comm_unique_id")
+        obj = [bytes(buf.raw)]
+        dist.broadcast_object_list(obj, src=0, group=group)
+        return obj[0]
+
     @classmethod
     def from_torch_distributed(cls, group=None) -> "Comm":
         import torch.distributed as dist
         rank, world = dist.get_rank(group), dist.get_world_size(group)
-        buf = ctypes.create_string_buffer(128)
-        if rank == 0:
-            _check(lib().ear_comm_unique_id(buf), "ear_comm_unique_id")
-        obj = [bytes(buf.raw)]
-        dist.broadcast_object_list(obj, src=0, group=group)
+        uid = cls.distribute_unique_id(group)
         h = _P()
-        _check(lib().ear_comm_init(obj[0], world, rank, ctypes.byref(h)), "ear_comm_init")
+        _check(lib().ear_comm_init(uid, world, rank, ctypes.byref(h)), "ear_comm_init")
         return cls(h, world, rank)
 
     def destroy(self):
@@ -218,6 +226,17 @@ def apsp_reduced(plan: Plan, D: torch.Tensor, comm: Comm | None = None, stream=N
     D = _dev_i32(D, "D")
     _check(lib().apsp_reduced(plan.handle, D.data_ptr(), D.stride(0), _comm_handle(comm), _stream(stream)),
            "apsp_reduced")
+    return D
+
+
+def apsp_reduced_emulated(plan: Plan, nranks: int, D: torch.Tensor | None = None, stream=None) -> torch.Tensor:
+    """The multi-GPU (row-block sharded) FW schedule for `nranks` ranks, emulated on this GPU."""
+    if D is None:
+        Np = plan.info(nranks).n_reduced_padded
+        D = torch.empty((Np, Np), dtype=torch.int32, device="cuda")
+    _dev_i32(D, "D")
+    _check(lib().apsp_reduced_emulated(plan.handle, nranks, D.data_ptr(), D.stride(0), _stream(stream)),
+           "apsp_reduced_emulated")
     return D
 
 
