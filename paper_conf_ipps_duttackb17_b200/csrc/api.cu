@@ -36,6 +36,21 @@ int32_t padded(const ear_plan_s *p, int32_t nranks) {
 
 bool aligned16(const void *p) { return ((uintptr_t)p & 15u) == 0; }
 
+// Scratch (D, sort buffers, pivot rows) comes from the device's default stream-ordered pool.  Keep
+// freed blocks cached instead of returning them to the driver at every synchronisation (the
+// default release threshold 0 would re-map the 3.6 GB D of cfg4 on every call).
+void ensure_pool() {
+  static bool done[64] = {false};
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64 || done[dev]) return;
+  cudaMemPool_t pool;
+  if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
+    uint64_t thr = UINT64_MAX;
+    cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+  }
+  done[dev] = true;
+}
+
 }  // namespace
 }  // namespace ear
 
@@ -75,6 +90,7 @@ ear_status_t ear_decompose(int32_t n, int64_t m, const int32_t *d_src, const int
     set_error("ear_decompose: bad sizes n=%d m=%lld", n, (long long)m);
     return EAR_EINVAL;
   }
+  ensure_pool();
   ear_plan_s *p = new ear_plan_s;
   cudaGetDevice(&p->device);
   int sp = prof_begin(PK_DECOMPOSE, (cudaStream_t)stream);

@@ -27,7 +27,7 @@ namespace {
 
 constexpr int NT = 256;
 constexpr int RB = 32;              // rows per CTA
-constexpr int ECAP = 24;            // endpoints per sub-group (R tile: ECAP x 1024 ints = 96 KB)
+constexpr int ECAP = 16;            // endpoints per sub-group (R tile: ECAP x 1024 ints = 64 KB)
 constexpr int CHUNK = NT * 4;       // columns per chunk
 constexpr int EXP_SMEM = ECAP * CHUNK * 4;
 
@@ -43,7 +43,7 @@ __device__ __forceinline__ int32_t out_val(int32_t cp, int32_t rp, int32_t cq, i
 }
 
 template <bool VEC>
-__global__ void __launch_bounds__(NT, 2) k_expand(const int32_t *__restrict__ D, int64_t ldd,
+__global__ void __launch_bounds__(NT, 3) k_expand(const int32_t *__restrict__ D, int64_t ldd,
                                                  const VDesc *__restrict__ desc, int32_t n, int32_t row_begin,
                                                  int32_t row_end, int32_t *__restrict__ out, int64_t ldo) {
   extern __shared__ __align__(16) int32_t R[];       // [ECAP][CHUNK]
@@ -105,14 +105,37 @@ __global__ void __launch_bounds__(NT, 2) k_expand(const int32_t *__restrict__ D,
     }
     for (int g = 0; g < nsg; ++g) {
       const int e0 = sg_e0[g], ne = sg_e0[g + 1] - e0;
-      for (int e = 0; e < ne; ++e) {
+      // R rows for the sub-group's endpoints; 4 endpoints per batch keep 32 independent gathers
+      // in flight per thread (the kernel is otherwise gather-latency bound)
+      int e = 0;
+      for (; e + 4 <= ne; e += 4) {
+        int32_t gp[4][4], gq[4][4];
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+          const int32_t *De = D + (int64_t)ends[e0 + e + u] * ldd;
+#pragma unroll
+          for (int j = 0; j < 4; ++j) {
+            gp[u][j] = __ldg(De + pt[j]);
+            gq[u][j] = __ldg(De + qt[j]);
+          }
+        }
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+          int4 v;   // clamped to INF so that cp_s + R below cannot overflow
+          v.x = min(__viaddmin_s32(gq[u][0], cqt[0], gp[u][0] + cpt[0]), INF);
+          v.y = min(__viaddmin_s32(gq[u][1], cqt[1], gp[u][1] + cpt[1]), INF);
+          v.z = min(__viaddmin_s32(gq[u][2], cqt[2], gp[u][2] + cpt[2]), INF);
+          v.w = min(__viaddmin_s32(gq[u][3], cqt[3], gp[u][3] + cpt[3]), INF);
+          *reinterpret_cast<int4 *>(Rt + (e + u) * CHUNK) = v;
+        }
+      }
+      for (; e < ne; ++e) {
         const int32_t *De = D + (int64_t)ends[e0 + e] * ldd;
         int4 v;
-        // clamp to INF so that cp_s + R below cannot overflow
-        v.x = min(__viaddmin_s32(De[qt[0]], cqt[0], De[pt[0]] + cpt[0]), INF);
-        v.y = min(__viaddmin_s32(De[qt[1]], cqt[1], De[pt[1]] + cpt[1]), INF);
-        v.z = min(__viaddmin_s32(De[qt[2]], cqt[2], De[pt[2]] + cpt[2]), INF);
-        v.w = min(__viaddmin_s32(De[qt[3]], cqt[3], De[pt[3]] + cpt[3]), INF);
+        v.x = min(__viaddmin_s32(__ldg(De + qt[0]), cqt[0], __ldg(De + pt[0]) + cpt[0]), INF);
+        v.y = min(__viaddmin_s32(__ldg(De + qt[1]), cqt[1], __ldg(De + pt[1]) + cpt[1]), INF);
+        v.z = min(__viaddmin_s32(__ldg(De + qt[2]), cqt[2], __ldg(De + pt[2]) + cpt[2]), INF);
+        v.w = min(__viaddmin_s32(__ldg(De + qt[3]), cqt[3], __ldg(De + pt[3]) + cpt[3]), INF);
         *reinterpret_cast<int4 *>(Rt + e * CHUNK) = v;
       }
       const int rend = sg_row0[g + 1];

@@ -15,8 +15,12 @@
 //   D[i,K] = D[K,i]^T: both operands are slices of the pivot ROW block, which is also the only
 //   block a multi-GPU round has to broadcast.  On one GPU only the upper triangle of tiles is
 //   computed and each result is written twice (tile and transposed mirror): half the min-plus work.
+#include <cuda.h>
+#include <cudaTypedefs.h>
+
 #include <algorithm>
 #include <cmath>
+#include <vector>
 
 #include "common.cuh"
 
@@ -27,7 +31,6 @@ constexpr int NT = 256;
 constexpr int KC = 32;                       // k-chunk depth
 constexpr int NCHUNK = TILE / KC;            // 4
 constexpr int SM_CHUNK = KC * TILE;          // ints per operand chunk (16 KB)
-constexpr int FW_SMEM = 2 * 2 * SM_CHUNK * 4; // 2 stages x 2 operands = 64 KB
 
 __global__ void k_init_D(int32_t *D, int64_t ldd, int32_t Np, int32_t row0, int32_t rows) {
   int64_t total = (int64_t)rows * (Np / 4);
@@ -107,41 +110,76 @@ __global__ void __launch_bounds__(NT, 1) k_fw_phase1(int32_t *T, int64_t ldt) {
 }
 
 // ------------------------------------------------------------------------------ phases 2 and 3
+// Persistent, TMA-fed min-plus tile kernel.  Each CTA walks its tiles (blockIdx.x, +gridDim.x, ...);
+// the operand chunks (A^T = P[k-rows][ti cols], B = P[k-rows][tj cols], 32 x 128 int32 each) stream
+// through a STAGES-deep shared-memory ring filled by cp.async.bulk.tensor (TMA) and guarded by
+// mbarriers (full: TMA bytes landed; empty: all 8 warps done reading), so no CTA-wide barrier sits
+// in the main loop and the next tile's first chunks are fetched while the current tile finishes.
+// Thread 0 doubles as the TMA producer.  The C tile lives in registers (8x8 per thread).
 enum { MODE_PIVOT_ROW = 0, MODE_UPPER = 1, MODE_ROWS = 2 };
+
+constexpr int STAGES = 3;
+constexpr int FW_SMEM = STAGES * 2 * SM_CHUNK * 4 + 2 * STAGES * 8;
 
 struct TileJob {
   int32_t *C;        // matrix holding the C tiles (local rows), leading dimension ldc
   int64_t ldc;
-  const int32_t *P;  // pivot row block: 128 rows x Np, leading dimension ldp
-  int64_t ldp;
+  int32_t p_row0;    // row coordinate of the pivot row block inside the operand tensor map
   int32_t k;         // pivot tile index
   int32_t nt;        // tiles per dimension (Np / 128)
   int32_t ti0;       // first local tile row (global index) of C
   int32_t nti;       // number of local tile rows
   int32_t mode;
   int32_t mirror;    // also write the transposed result into tile (tj, ti) (single GPU)
+  int64_t ntiles;    // tiles in this launch
 };
 
-__device__ __forceinline__ void cp_async16(void *smem, const void *gmem) {
-  unsigned s = (unsigned)__cvta_generic_to_shared(smem);
-  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(s), "l"(gmem));
-}
-__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::); }
-template <int N>
-__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;\n" ::"n"(N)); }
+__device__ __forceinline__ uint32_t smem_u32(const void *p) { return (uint32_t)__cvta_generic_to_shared(p); }
 
-// decode the CTA index into (ti, tj)
-__device__ __forceinline__ bool decode_tile(const TileJob &J, int64_t idx, int &ti, int &tj) {
+__device__ __forceinline__ void mbar_init(uint64_t *b, uint32_t cnt) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;\n" ::"r"(smem_u32(b)), "r"(cnt) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t *b) {
+  asm volatile("{\n\t.reg .b64 st;\n\tmbarrier.arrive.shared::cta.b64 st, [%0];\n\t}\n" ::"r"(smem_u32(b)) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive_tx(uint64_t *b, uint32_t bytes) {
+  asm volatile("{\n\t.reg .b64 st;\n\tmbarrier.arrive.expect_tx.shared::cta.b64 st, [%0], %1;\n\t}\n" ::"r"(smem_u32(b)),
+               "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ bool mbar_try(uint64_t *b, uint32_t parity) {
+  uint32_t ok;
+  asm volatile(
+      "{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\tselp.u32 %0, 1, 0, p;\n\t}\n"
+      : "=r"(ok)
+      : "r"(smem_u32(b)), "r"(parity)
+      : "memory");
+  return ok != 0;
+}
+__device__ __forceinline__ void mbar_wait(uint64_t *b, uint32_t parity) {
+  while (!mbar_try(b, parity)) {
+  }
+}
+__device__ __forceinline__ void tma_load_2d(void *dst, const CUtensorMap *map, int32_t c0, int32_t c1, uint64_t *bar) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];\n" ::"r"(
+          smem_u32(dst)),
+      "l"(reinterpret_cast<uint64_t>(map)), "r"(c0), "r"(c1), "r"(smem_u32(bar))
+      : "memory");
+}
+
+// decode the tile index into (ti, tj)
+__device__ __forceinline__ void decode_tile(const TileJob &J, int64_t idx, int &ti, int &tj) {
   const int k = J.k;
   if (J.mode == MODE_PIVOT_ROW) {
     ti = k;
     tj = (int)idx < k ? (int)idx : (int)idx + 1;
-    return true;
+    return;
   }
   if (J.mode == MODE_UPPER) {
-    // upper triangle (a <= b) of the (nt-1) x (nt-1) non-pivot tiles, row-major
+    // upper triangle (a <= b) of the (nt-1) x (nt-1) non-pivot tiles, row-major; row a starts at
+    // a*T - a*(a-1)/2
     const int64_t T = J.nt - 1;
-    // a = largest a with a*T - a*(a-1)/2 <= idx
     double tt = (double)(2 * T + 1);
     int64_t a = (int64_t)floor((tt - sqrt(tt * tt - 8.0 * (double)idx)) * 0.5);
     if (a < 0) a = 0;
@@ -150,7 +188,7 @@ __device__ __forceinline__ bool decode_tile(const TileJob &J, int64_t idx, int &
     const int64_t b = a + (idx - (a * T - a * (a - 1) / 2));
     ti = (int)a < k ? (int)a : (int)a + 1;
     tj = (int)b < k ? (int)b : (int)b + 1;
-    return true;
+    return;
   }
   // MODE_ROWS: local tile rows except the pivot row, all columns except the pivot column
   const int64_t ncols = J.nt - 1;
@@ -158,87 +196,97 @@ __device__ __forceinline__ bool decode_tile(const TileJob &J, int64_t idx, int &
   ti = J.ti0 + r;
   if (ti >= k && k >= J.ti0 && k < J.ti0 + J.nti) ti++;   // skip the pivot tile row if local
   tj = cidx < k ? cidx : cidx + 1;
-  return true;
 }
 
-__global__ void __launch_bounds__(NT, 2) k_fw_tiles(TileJob J) {
-  extern __shared__ __align__(16) int32_t smem[];
-  int32_t *sA = smem;                       // [2][KC][TILE]   A^T chunk = P[k-rows][ti cols]
-  int32_t *sB = smem + 2 * SM_CHUNK;        // [2][KC][TILE]   B chunk   = P[k-rows][tj cols]
-  const int tid = threadIdx.x;
+__global__ void __launch_bounds__(NT, 2) k_fw_tiles(const __grid_constant__ CUtensorMap tmP, const TileJob J) {
+  extern __shared__ __align__(128) int32_t smem[];
+  int32_t *sA = smem;                                   // [STAGES][KC][TILE]   A^T chunks
+  int32_t *sB = smem + STAGES * SM_CHUNK;               // [STAGES][KC][TILE]   B chunks
+  uint64_t *full = reinterpret_cast<uint64_t *>(smem + 2 * STAGES * SM_CHUNK);
+  uint64_t *empty = full + STAGES;
+  const int tid = threadIdx.x, lane = tid & 31;
   const int tx = tid & 15, ty = tid >> 4;
-  int ti, tj;
-  decode_tile(J, blockIdx.x, ti, tj);
 
-  const int32_t *pa = J.P + (int64_t)ti * TILE;
-  const int32_t *pb = J.P + (int64_t)tj * TILE;
-  auto load_chunk = [&](int kc, int stage) {
-#pragma unroll
-    for (int it = 0; it < 4; ++it) {
-      const int piece = tid + it * NT;           // 0..1023: 32 rows x 32 pieces of 16 B
-      const int rr = piece >> 5, cc = (piece & 31) * 4;
-      const int64_t goff = (int64_t)(kc * KC + rr) * J.ldp + cc;
-      cp_async16(sA + stage * SM_CHUNK + rr * TILE + cc, pa + goff);
-      cp_async16(sB + stage * SM_CHUNK + rr * TILE + cc, pb + goff);
+  if (tid == 0) {
+    for (int s = 0; s < STAGES; ++s) {
+      mbar_init(&full[s], 1);
+      mbar_init(&empty[s], NT / 32);
     }
-    cp_async_commit();
+    asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
+    asm volatile("prefetch.tensormap [%0];\n" ::"l"(reinterpret_cast<uint64_t>(&tmP)) : "memory");
+  }
+  __syncthreads();
+
+  const int64_t my_tiles = J.ntiles > (int64_t)blockIdx.x ? (J.ntiles - 1 - blockIdx.x) / gridDim.x + 1 : 0;
+  const int64_t total_chunks = my_tiles * NCHUNK;
+  int64_t issued = 0;   // producer state (thread 0 only)
+  auto produce = [&](int64_t upto) {
+    while (issued < upto) {
+      const int st = (int)(issued % STAGES);
+      if (issued >= STAGES) mbar_wait(&empty[st], (uint32_t)((issued / STAGES - 1) & 1));
+      int pti, ptj;
+      decode_tile(J, blockIdx.x + (issued / NCHUNK) * gridDim.x, pti, ptj);
+      const int row = J.p_row0 + (int)(issued % NCHUNK) * KC;
+      mbar_arrive_tx(&full[st], 2 * SM_CHUNK * 4);
+      tma_load_2d(sA + st * SM_CHUNK, &tmP, pti * TILE, row, &full[st]);
+      tma_load_2d(sB + st * SM_CHUNK, &tmP, ptj * TILE, row, &full[st]);
+      ++issued;
+    }
   };
-  load_chunk(0, 0);
+  if (tid == 0) produce(total_chunks < STAGES ? total_chunks : STAGES);
 
-  // C tile -> registers
-  int32_t *Ct = J.C + (int64_t)(ti - J.ti0) * TILE * J.ldc + (int64_t)tj * TILE;
-  int32_t c[8][8];
+  int64_t g = 0;   // chunk counter (all threads)
+  for (int64_t it = 0; it < my_tiles; ++it) {
+    int ti, tj;
+    decode_tile(J, blockIdx.x + it * gridDim.x, ti, tj);
+    int32_t *Ct = J.C + (int64_t)(ti - J.ti0) * TILE * J.ldc + (int64_t)tj * TILE;
+    int32_t c[8][8];
 #pragma unroll
-  for (int r = 0; r < 8; ++r) {
-    const int i = (r < 4 ? 0 : 64) + ty * 4 + (r & 3);
-    const int4 lo = *reinterpret_cast<const int4 *>(Ct + (int64_t)i * J.ldc + tx * 4);
-    const int4 hi = *reinterpret_cast<const int4 *>(Ct + (int64_t)i * J.ldc + 64 + tx * 4);
-    c[r][0] = lo.x; c[r][1] = lo.y; c[r][2] = lo.z; c[r][3] = lo.w;
-    c[r][4] = hi.x; c[r][5] = hi.y; c[r][6] = hi.z; c[r][7] = hi.w;
-  }
-
+    for (int r = 0; r < 8; ++r) {
+      const int i = (r < 4 ? 0 : 64) + ty * 4 + (r & 3);
+      const int4 lo = *reinterpret_cast<const int4 *>(Ct + (int64_t)i * J.ldc + tx * 4);
+      const int4 hi = *reinterpret_cast<const int4 *>(Ct + (int64_t)i * J.ldc + 64 + tx * 4);
+      c[r][0] = lo.x; c[r][1] = lo.y; c[r][2] = lo.z; c[r][3] = lo.w;
+      c[r][4] = hi.x; c[r][5] = hi.y; c[r][6] = hi.z; c[r][7] = hi.w;
+    }
 #pragma unroll 1
-  for (int kc = 0; kc < NCHUNK; ++kc) {
-    const int stage = kc & 1;
-    if (kc + 1 < NCHUNK) {
-      load_chunk(kc + 1, stage ^ 1);
-      cp_async_wait<1>();
-    } else {
-      cp_async_wait<0>();
-    }
-    __syncthreads();
-    const int32_t *a_s = sA + stage * SM_CHUNK;
-    const int32_t *b_s = sB + stage * SM_CHUNK;
+    for (int kc = 0; kc < NCHUNK; ++kc, ++g) {
+      if (tid == 0) produce(g + STAGES < total_chunks ? g + STAGES : total_chunks);
+      const int st = (int)(g % STAGES);
+      mbar_wait(&full[st], (uint32_t)((g / STAGES) & 1));
+      const int32_t *a_s = sA + st * SM_CHUNK;
+      const int32_t *b_s = sB + st * SM_CHUNK;
 #pragma unroll 4
-    for (int kk = 0; kk < KC; ++kk) {
-      const int4 alo = *reinterpret_cast<const int4 *>(a_s + kk * TILE + ty * 4);
-      const int4 ahi = *reinterpret_cast<const int4 *>(a_s + kk * TILE + 64 + ty * 4);
-      const int4 blo = *reinterpret_cast<const int4 *>(b_s + kk * TILE + tx * 4);
-      const int4 bhi = *reinterpret_cast<const int4 *>(b_s + kk * TILE + 64 + tx * 4);
-      const int32_t a[8] = {alo.x, alo.y, alo.z, alo.w, ahi.x, ahi.y, ahi.z, ahi.w};
-      const int32_t b[8] = {blo.x, blo.y, blo.z, blo.w, bhi.x, bhi.y, bhi.z, bhi.w};
+      for (int kk = 0; kk < KC; ++kk) {
+        const int4 alo = *reinterpret_cast<const int4 *>(a_s + kk * TILE + ty * 4);
+        const int4 ahi = *reinterpret_cast<const int4 *>(a_s + kk * TILE + 64 + ty * 4);
+        const int4 blo = *reinterpret_cast<const int4 *>(b_s + kk * TILE + tx * 4);
+        const int4 bhi = *reinterpret_cast<const int4 *>(b_s + kk * TILE + 64 + tx * 4);
+        const int32_t a[8] = {alo.x, alo.y, alo.z, alo.w, ahi.x, ahi.y, ahi.z, ahi.w};
+        const int32_t b[8] = {blo.x, blo.y, blo.z, blo.w, bhi.x, bhi.y, bhi.z, bhi.w};
 #pragma unroll
-      for (int r = 0; r < 8; ++r)
+        for (int r = 0; r < 8; ++r)
 #pragma unroll
-        for (int q = 0; q < 8; ++q) c[r][q] = mp(a[r], b[q], c[r][q]);
+          for (int q = 0; q < 8; ++q) c[r][q] = mp(a[r], b[q], c[r][q]);
+      }
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&empty[st]);
     }
-    __syncthreads();
-  }
-
-  // epilogue: tile, and (single GPU, off-diagonal) its transposed mirror
+    // epilogue: tile, and (single GPU, off-diagonal) its transposed mirror
 #pragma unroll
-  for (int r = 0; r < 8; ++r) {
-    const int i = (r < 4 ? 0 : 64) + ty * 4 + (r & 3);
-    *reinterpret_cast<int4 *>(Ct + (int64_t)i * J.ldc + tx * 4) = make_int4(c[r][0], c[r][1], c[r][2], c[r][3]);
-    *reinterpret_cast<int4 *>(Ct + (int64_t)i * J.ldc + 64 + tx * 4) = make_int4(c[r][4], c[r][5], c[r][6], c[r][7]);
-  }
-  if (J.mirror && ti != tj) {
-    int32_t *Mt = J.C + (int64_t)tj * TILE * J.ldc + (int64_t)ti * TILE;
+    for (int r = 0; r < 8; ++r) {
+      const int i = (r < 4 ? 0 : 64) + ty * 4 + (r & 3);
+      *reinterpret_cast<int4 *>(Ct + (int64_t)i * J.ldc + tx * 4) = make_int4(c[r][0], c[r][1], c[r][2], c[r][3]);
+      *reinterpret_cast<int4 *>(Ct + (int64_t)i * J.ldc + 64 + tx * 4) = make_int4(c[r][4], c[r][5], c[r][6], c[r][7]);
+    }
+    if (J.mirror && ti != tj) {
+      int32_t *Mt = J.C + (int64_t)tj * TILE * J.ldc + (int64_t)ti * TILE;
 #pragma unroll
-    for (int q = 0; q < 8; ++q) {
-      const int j = (q < 4 ? 0 : 64) + tx * 4 + (q & 3);
-      *reinterpret_cast<int4 *>(Mt + (int64_t)j * J.ldc + ty * 4) = make_int4(c[0][q], c[1][q], c[2][q], c[3][q]);
-      *reinterpret_cast<int4 *>(Mt + (int64_t)j * J.ldc + 64 + ty * 4) = make_int4(c[4][q], c[5][q], c[6][q], c[7][q]);
+      for (int q = 0; q < 8; ++q) {
+        const int j = (q < 4 ? 0 : 64) + tx * 4 + (q & 3);
+        *reinterpret_cast<int4 *>(Mt + (int64_t)j * J.ldc + ty * 4) = make_int4(c[0][q], c[1][q], c[2][q], c[3][q]);
+        *reinterpret_cast<int4 *>(Mt + (int64_t)j * J.ldc + 64 + ty * 4) = make_int4(c[4][q], c[5][q], c[6][q], c[7][q]);
+      }
     }
   }
 }
@@ -261,14 +309,48 @@ __global__ void k_col_tiles_from_pivot(int32_t *C, int64_t ldc, const int32_t *P
 }
 
 bool g_smem_set = false;
+int g_num_sms = 0;
+PFN_cuTensorMapEncodeTiled_v12000 g_encode = nullptr;
 
-ear_status_t launch_tiles(const TileJob &J, int64_t nblocks, cudaStream_t st) {
+// 2-D int32 tensor map over rows x cols (leading dimension ld elements) with a 32 x 128 box
+ear_status_t make_map(CUtensorMap *map, const int32_t *base, int64_t rows, int64_t cols, int64_t ld) {
+  if (!g_encode) {
+    cudaDriverEntryPointQueryResult q;
+    void *fn = nullptr;
+    EAR_CUDA_TRY(cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q));
+    if (!fn || q != cudaDriverEntryPointSuccess) {
+      set_error("cuTensorMapEncodeTiled unavailable");
+      return EAR_ECUDA;
+    }
+    g_encode = (PFN_cuTensorMapEncodeTiled_v12000)fn;
+  }
+  cuuint64_t dims[2] = {(cuuint64_t)cols, (cuuint64_t)rows};
+  cuuint64_t strides[1] = {(cuuint64_t)ld * sizeof(int32_t)};
+  cuuint32_t box[2] = {(cuuint32_t)TILE, (cuuint32_t)KC};
+  cuuint32_t estr[2] = {1, 1};
+  CUresult r = g_encode(map, CU_TENSOR_MAP_DATA_TYPE_INT32, 2, (void *)base, dims, strides, box, estr,
+                        CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                        CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) {
+    set_error("cuTensorMapEncodeTiled failed (%d) rows=%lld cols=%lld ld=%lld", (int)r, (long long)rows,
+              (long long)cols, (long long)ld);
+    return EAR_ECUDA;
+  }
+  return EAR_OK;
+}
+
+ear_status_t launch_tiles(const CUtensorMap &map, TileJob J, int64_t nblocks, cudaStream_t st) {
   if (!g_smem_set) {
     EAR_CUDA_TRY(cudaFuncSetAttribute(k_fw_tiles, cudaFuncAttributeMaxDynamicSharedMemorySize, FW_SMEM));
+    int dev = 0;
+    EAR_CUDA_TRY(cudaGetDevice(&dev));
+    EAR_CUDA_TRY(cudaDeviceGetAttribute(&g_num_sms, cudaDevAttrMultiProcessorCount, dev));
     g_smem_set = true;
   }
   if (nblocks <= 0) return EAR_OK;
-  EAR_LAUNCH(k_fw_tiles, (unsigned)nblocks, NT, FW_SMEM, st)(J);
+  J.ntiles = nblocks;
+  const int64_t grid = std::min<int64_t>(nblocks, (int64_t)g_num_sms * 2);   // persistent: 2 CTAs / SM
+  EAR_LAUNCH(k_fw_tiles, (unsigned)grid, NT, FW_SMEM, st)(map, J);
   return EAR_OK;
 }
 
@@ -293,19 +375,21 @@ ear_status_t fw_init_D(const ear_plan_s *plan, int32_t *D, int64_t ldd, int32_t 
 ear_status_t fw_single(int32_t *D, int64_t ldd, int32_t Np, cudaStream_t st) {
   const int nt = Np / TILE;
   const double tile_ops = (double)TILE * TILE * TILE;
+  CUtensorMap map;
+  EAR_TRY(make_map(&map, D, Np, Np, ldd));
   for (int k = 0; k < nt; ++k) {
     int32_t *Pk = D + (int64_t)k * TILE * ldd;            // pivot row block
     int s1 = prof_begin(PK_FW_P1, st);
     EAR_LAUNCH(k_fw_phase1, 1, NT, 0, st)(Pk + (int64_t)k * TILE, ldd);
     prof_end(s1, st, tile_ops);
-    TileJob J{D, ldd, Pk, ldd, k, nt, 0, nt, MODE_PIVOT_ROW, 1};
+    TileJob J{D, ldd, k * TILE, k, nt, 0, nt, MODE_PIVOT_ROW, 1, 0};
     int s2 = prof_begin(PK_FW_P2, st);
-    EAR_TRY(launch_tiles(J, nt - 1, st));
+    EAR_TRY(launch_tiles(map, J, nt - 1, st));
     prof_end(s2, st, (nt - 1) * tile_ops);
     J.mode = MODE_UPPER;
     const int64_t nup = (int64_t)(nt - 1) * nt / 2;
     int s3 = prof_begin(PK_FW_P3, st);
-    EAR_TRY(launch_tiles(J, nup, st));
+    EAR_TRY(launch_tiles(map, J, nup, st));
     prof_end(s3, st, nup * tile_ops);
   }
   EAR_CUDA_TRY(cudaGetLastError());
@@ -322,13 +406,16 @@ struct ShardCtx {
   int64_t ldd;
   int32_t Np, nt, P, rank, nti, ti0;
   int32_t *prow;    // 128 x Np pivot row block (leading dimension Np)
+  CUtensorMap map_blk, map_prow;
 };
 
-static ShardCtx shard_ctx(int32_t *Dblk, int64_t ldd, int32_t Np, int32_t P, int32_t rank, int32_t *prow) {
-  ShardCtx c;
-  c.Dblk = Dblk; c.ldd = ldd; c.Np = Np; c.nt = Np / TILE; c.P = P; c.rank = rank;
-  c.nti = c.nt / P; c.ti0 = rank * c.nti; c.prow = prow;
-  return c;
+static ear_status_t shard_ctx(ShardCtx *c, int32_t *Dblk, int64_t ldd, int32_t Np, int32_t P, int32_t rank,
+                              int32_t *prow) {
+  c->Dblk = Dblk; c->ldd = ldd; c->Np = Np; c->nt = Np / TILE; c->P = P; c->rank = rank;
+  c->nti = c->nt / P; c->ti0 = rank * c->nti; c->prow = prow;
+  EAR_TRY(make_map(&c->map_blk, Dblk, (int64_t)c->nti * TILE, Np, ldd));
+  EAR_TRY(make_map(&c->map_prow, prow, TILE, Np, Np));
+  return EAR_OK;
 }
 
 static ear_status_t shard_owner_step(const ShardCtx &c, int k, cudaStream_t st) {
@@ -338,9 +425,9 @@ static ear_status_t shard_owner_step(const ShardCtx &c, int k, cudaStream_t st) 
   EAR_LAUNCH(k_fw_phase1, 1, NT, 0, st)(Pk + (int64_t)k * TILE, c.ldd);
   prof_end(s1, st, tile_ops);
   // pivot-row tiles; C rows are the pivot rows themselves (ti0 = k: local row offset 0)
-  TileJob J{Pk, c.ldd, Pk, c.ldd, k, c.nt, k, 1, MODE_PIVOT_ROW, 0};
+  TileJob J{Pk, c.ldd, (k - c.ti0) * TILE, k, c.nt, k, 1, MODE_PIVOT_ROW, 0, 0};
   int s2 = prof_begin(PK_FW_P2, st);
-  EAR_TRY(launch_tiles(J, c.nt - 1, st));
+  EAR_TRY(launch_tiles(c.map_blk, J, c.nt - 1, st));
   prof_end(s2, st, (c.nt - 1) * tile_ops);
   EAR_CUDA_TRY(cudaMemcpy2DAsync(c.prow, sizeof(int32_t) * c.Np, Pk, sizeof(int32_t) * c.ldd,
                                  sizeof(int32_t) * c.Np, TILE, cudaMemcpyDeviceToDevice, st));
@@ -353,9 +440,9 @@ static ear_status_t shard_update_step(const ShardCtx &c, int k, cudaStream_t st)
   dim3 g(16, c.nti);
   EAR_LAUNCH(k_col_tiles_from_pivot, g, 256, 0, st)(c.Dblk, c.ldd, c.prow, c.Np, k, c.ti0, c.nti);
   const int rows_here = (owner == c.rank) ? c.nti - 1 : c.nti;
-  TileJob J{c.Dblk, c.ldd, c.prow, c.Np, k, c.nt, c.ti0, c.nti, MODE_ROWS, 0};
+  TileJob J{c.Dblk, c.ldd, 0, k, c.nt, c.ti0, c.nti, MODE_ROWS, 0, 0};
   int s3 = prof_begin(PK_FW_P3, st);
-  EAR_TRY(launch_tiles(J, (int64_t)rows_here * (c.nt - 1), st));
+  EAR_TRY(launch_tiles(c.map_prow, J, (int64_t)rows_here * (c.nt - 1), st));
   prof_end(s3, st, (double)rows_here * (c.nt - 1) * tile_ops);
   return EAR_OK;
 }
@@ -363,8 +450,8 @@ static ear_status_t shard_update_step(const ShardCtx &c, int k, cudaStream_t st)
 ear_status_t fw_sharded(int32_t *Dblk, int64_t ldd, int32_t Np, ear_comm_s *comm, cudaStream_t st) {
   int32_t *prow = nullptr;
   EAR_CUDA_TRY(cudaMallocAsync((void **)&prow, sizeof(int32_t) * (size_t)TILE * Np, st));
-  const ShardCtx c = shard_ctx(Dblk, ldd, Np, comm->nranks, comm->rank, prow);
-  ear_status_t status = EAR_OK;
+  ShardCtx c;
+  ear_status_t status = shard_ctx(&c, Dblk, ldd, Np, comm->nranks, comm->rank, prow);
   for (int k = 0; k < c.nt && status == EAR_OK; ++k) {
     const int owner = k / c.nti;
     if (owner == c.rank) status = shard_owner_step(c, k, st);
@@ -390,11 +477,13 @@ ear_status_t fw_sharded_emulated(int32_t *D, int64_t ldd, int32_t Np, int32_t P,
   const int32_t R = Np / P;
   ear_status_t status = EAR_OK;
   const int nt = Np / TILE, nti = nt / P;
+  std::vector<ShardCtx> ctx(P);
+  for (int r = 0; r < P && status == EAR_OK; ++r)
+    status = shard_ctx(&ctx[r], D + (int64_t)r * R * ldd, ldd, Np, P, r, prow);
   for (int k = 0; k < nt && status == EAR_OK; ++k) {
     const int owner = k / nti;
-    status = shard_owner_step(shard_ctx(D + (int64_t)owner * R * ldd, ldd, Np, P, owner, prow), k, st);
-    for (int r = 0; r < P && status == EAR_OK; ++r)
-      status = shard_update_step(shard_ctx(D + (int64_t)r * R * ldd, ldd, Np, P, r, prow), k, st);
+    status = shard_owner_step(ctx[owner], k, st);
+    for (int r = 0; r < P && status == EAR_OK; ++r) status = shard_update_step(ctx[r], k, st);
   }
   cudaFreeAsync(prow, st);
   if (status != EAR_OK) return status;
