@@ -98,6 +98,8 @@ ear_status_t ear_plan_export(ear_plan_t plan, int32_t *d_tid, int32_t *d_ear, in
 ear_status_t ear_plan_export_reduced_edges(ear_plan_t plan, int32_t *d_u, int32_t *d_v, int32_t *d_w,
                                            void *stream);
 
+/* Release a plan.  Its device arrays come from the device's stream-ordered memory pool and are freed
+ * in stream order on the stream given to ear_decompose, which must still be valid. */
 void ear_plan_destroy(ear_plan_t plan);
 
 /* ---------------------------------------------------------------- Phase II: APSP(G^r)
@@ -141,6 +143,14 @@ ear_status_t ear_gather_reduced(ear_plan_t plan, const int32_t *d_D_block, int64
  * path).  Asynchronous.  Errors: EAR_EINVAL (range, ldo < n, ldd), EAR_ECUDA. */
 ear_status_t expand_ears(ear_plan_t plan, const int32_t *d_D_full, int64_t ldd, int32_t row_begin,
                          int32_t row_end, int32_t *d_out, int64_t ldo, void *stream);
+
+/* Compact / query mode (the paper's storage argument, P:137 and Table 1 "Our's
+ * memory"): S[d_s[i], d_t[i]] for npairs arbitrary pairs, evaluated per pair from the full D and the
+ * plan's descriptors with the same rules as expand_ears -- O(N_r^2 + N) memory instead of
+ * the N^2 matrix.  d_s, d_t: DEVICE int32 vertex ids in [0,n) (not validated: out-of-range ids are
+ * undefined behaviour); d_out: DEVICE int32[npairs].  Asynchronous.  Errors: EAR_EINVAL. */
+ear_status_t ear_query_pairs(ear_plan_t plan, const int32_t *d_D_full, int64_t ldd, int64_t npairs,
+                             const int32_t *d_s, const int32_t *d_t, int32_t *d_out, void *stream);
 
 /* ---------------------------------------------------------------- Everything: Algorithm 1
  * APSP(G): ear_decompose + apsp_reduced (+ all-gather with comm) + expand_ears into rows

@@ -6,4 +6,4 @@ seeded synthetic workloads.  There is no CPU fallback.
 """
 from .ear_apsp import (FLAG_NO_CONTRACT, FLAG_NONE, INF, TILE, Comm, EarError, Plan, alloc_D, apsp_full,  # noqa: F401
                        apsp_full_host, apsp_reduced, apsp_reduced_emulated, ear_decompose, expand_ears, gather_reduced, lib, profile_enable,
-                       profile_read, profile_reset, row_block, version)
+                       profile_read, profile_reset, query_pairs, row_block, version)

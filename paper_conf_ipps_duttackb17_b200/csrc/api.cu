@@ -227,6 +227,16 @@ ear_status_t expand_ears(ear_plan_t p, const int32_t *d_D_full, int64_t ldd, int
   return expand(p, d_D_full, ldd, row_begin, row_end, d_out, ldo, (cudaStream_t)stream);
 }
 
+ear_status_t ear_query_pairs(ear_plan_t p, const int32_t *d_D_full, int64_t ldd, int64_t npairs, const int32_t *d_s,
+                             const int32_t *d_t, int32_t *d_out, void *stream) {
+  g_err[0] = 0;
+  if (!p || !d_D_full || npairs < 0 || (npairs > 0 && (!d_s || !d_t || !d_out)) || ldd < p->n_reduced) {
+    set_error("ear_query_pairs: bad argument");
+    return EAR_EINVAL;
+  }
+  return query_pairs(p, d_D_full, ldd, npairs, d_s, d_t, d_out, (cudaStream_t)stream);
+}
+
 // Phases II + III for an existing plan into device rows (shared by apsp_full / apsp_full_host).
 static ear_status_t solve_rows(ear_plan_s *p, int32_t row_begin, int32_t row_end, int32_t *d_out, int64_t ldo,
                                ear_comm_t comm, cudaStream_t st, int32_t **D_keep) {

@@ -53,6 +53,7 @@ struct ear_plan_s {
   int64_t n_redges = 0;
   uint32_t flags = 0;
   int device = 0;
+  cudaStream_t stream = nullptr;   // creation stream; plan arrays are freed on it (stream order)
   // per vertex
   ear::VDesc *desc = nullptr;  // [n]
   int32_t *tid = nullptr;      // [n] terminal id or -1
@@ -95,6 +96,8 @@ ear_status_t fw_sharded_emulated(int32_t *D, int64_t ldd, int32_t Np, int32_t P,
 // expand.cu
 ear_status_t expand(const ear_plan_s *plan, const int32_t *D, int64_t ldd, int32_t row_begin,
                     int32_t row_end, int32_t *out, int64_t ldo, cudaStream_t stream);
+ear_status_t query_pairs(const ear_plan_s *plan, const int32_t *D, int64_t ldd, int64_t npairs, const int32_t *qs,
+                         const int32_t *qt, int32_t *out, cudaStream_t stream);
 // comm.cu
 ear_status_t comm_bcast(ear_comm_s *comm, int32_t *buf, int64_t count, int32_t root, cudaStream_t stream);
 ear_status_t comm_allgather(ear_comm_s *comm, const int32_t *send, int32_t *recv, int64_t count,

@@ -295,19 +295,21 @@ struct Scratch {
 
 }  // namespace
 
+// Plan arrays come from the device's stream-ordered pool (cached; no driver call in steady state)
+// and are released in stream order on the stream the plan was created on.
 void plan_free(ear_plan_s *p) {
   if (!p) return;
   void *arrs[] = {p->desc, p->tid, p->ear, p->seg_of, p->seg_start, p->seg_vert, p->re_u, p->re_v, p->re_w};
   for (void *a : arrs)
-    if (a) cudaFree(a);
+    if (a) cudaFreeAsync(a, p->stream);
 }
 
 template <class T>
-static ear_status_t plan_alloc(T **p, int64_t count) {
+static ear_status_t plan_alloc(T **p, int64_t count, cudaStream_t st) {
   if (count <= 0) count = 1;
-  cudaError_t e = cudaMalloc((void **)p, sizeof(T) * (size_t)count);
+  cudaError_t e = cudaMallocAsync((void **)p, sizeof(T) * (size_t)count, st);
   if (e != cudaSuccess) {
-    set_error("cudaMalloc: %s", cudaGetErrorString(e));
+    set_error("cudaMallocAsync: %s", cudaGetErrorString(e));
     return EAR_ENOMEM;
   }
   return EAR_OK;
@@ -317,6 +319,7 @@ ear_status_t decompose(int32_t n, int64_t m, const int32_t *src, const int32_t *
                        uint32_t flags, cudaStream_t st, ear_plan_s *plan) {
   plan->n = n;
   plan->flags = flags;
+  plan->stream = st;
   Scratch S{st, {}};
 
   // ---- validation (reads the flags back at the N_r synchronisation point below; an invalid input
@@ -453,10 +456,10 @@ ear_status_t decompose(int32_t n, int64_t m, const int32_t *src, const int32_t *
   EAR_CUDA_TRY(cudaMemcpyAsync(&h_last[1], term + n - 1, sizeof(int32_t), cudaMemcpyDeviceToHost, st));
 
   // descriptors
-  EAR_TRY(plan_alloc(&plan->desc, n));
-  EAR_TRY(plan_alloc(&plan->tid, n));
-  EAR_TRY(plan_alloc(&plan->ear, n));
-  EAR_TRY(plan_alloc(&plan->seg_of, n));
+  EAR_TRY(plan_alloc(&plan->desc, n, st));
+  EAR_TRY(plan_alloc(&plan->tid, n, st));
+  EAR_TRY(plan_alloc(&plan->ear, n, st));
+  EAR_TRY(plan_alloc(&plan->seg_of, n, st));
   int32_t *ear_cnt, *d_stats;
   uint64_t *seg_key, *seg_key2;
   int32_t *seg_val, *seg_val2;
@@ -484,9 +487,9 @@ ear_status_t decompose(int32_t n, int64_t m, const int32_t *src, const int32_t *
   plan->n_chains = h_stats[0];
   plan->max_chain_len = h_stats[1];
   plan->n_redges = (int64_t)h_rcount;
-  EAR_TRY(plan_alloc(&plan->re_u, plan->n_redges));
-  EAR_TRY(plan_alloc(&plan->re_v, plan->n_redges));
-  EAR_TRY(plan_alloc(&plan->re_w, plan->n_redges));
+  EAR_TRY(plan_alloc(&plan->re_u, plan->n_redges, st));
+  EAR_TRY(plan_alloc(&plan->re_v, plan->n_redges, st));
+  EAR_TRY(plan_alloc(&plan->re_w, plan->n_redges, st));
   EAR_CUDA_TRY(cudaMemsetAsync(d_rcount, 0, sizeof(unsigned long long), st));
   if (A > 0)
     EAR_LAUNCH(k_reduced_arcs, grid_for(A), NT, 0, st)(A, asrc, term, scan, rb[cur], plan->re_u, plan->re_v, plan->re_w,
@@ -495,8 +498,8 @@ ear_status_t decompose(int32_t n, int64_t m, const int32_t *src, const int32_t *
   // same-chain vertex lists sorted by (chain id, off_left)
   const int32_t nc = n - plan->n_reduced;
   plan->n_chain_vertices = nc;
-  EAR_TRY(plan_alloc(&plan->seg_start, (int64_t)plan->n_chains + 1));
-  EAR_TRY(plan_alloc(&plan->seg_vert, nc));
+  EAR_TRY(plan_alloc(&plan->seg_start, (int64_t)plan->n_chains + 1, st));
+  EAR_TRY(plan_alloc(&plan->seg_vert, nc, st));
   if (nc > 0) {
     size_t tb = 0;
     cub::DoubleBuffer<uint64_t> dk(seg_key, seg_key2);

@@ -139,10 +139,16 @@ __global__ void __launch_bounds__(NT, 3) k_expand(const int32_t *__restrict__ D,
         *reinterpret_cast<int4 *>(Rt + e * CHUNK) = v;
       }
       const int rend = sg_row0[g + 1];
+      int last_p = -1, last_q = -1;
+      int4 a = make_int4(0, 0, 0, 0), b = a;
       for (int r = sg_row0[g]; r < rend; ++r) {
         const VDesc s = rdesc[r];
-        const int4 a = *reinterpret_cast<const int4 *>(Rt + ip[r] * CHUNK);
-        const int4 b = *reinterpret_cast<const int4 *>(Rt + iq[r] * CHUNK);
+        const int rp = ip[r], rq = iq[r];
+        if (rp != last_p || rq != last_q) {   // consecutive rows of one chain share their R rows
+          a = *reinterpret_cast<const int4 *>(Rt + rp * CHUNK);
+          b = (rq == rp) ? a : *reinterpret_cast<const int4 *>(Rt + rq * CHUNK);   // terminal rows: one load
+          last_p = rp; last_q = rq;
+        }
         int4 o;
         o.x = out_val(s.cp, a.x, s.cq, b.x);
         o.y = out_val(s.cp, a.y, s.cq, b.y);
@@ -182,6 +188,26 @@ __global__ void k_same_chain(const VDesc *__restrict__ desc, const int32_t *__re
   }
 }
 
+// Compact / query mode: S[s,t] for arbitrary pairs from D and the descriptors
+// alone -- UPDATE_DISTANCE evaluated per pair, O(N_r^2 + N) memory instead of N^2.
+__global__ void k_query_pairs(const int32_t *__restrict__ D, int64_t ldd, const VDesc *__restrict__ desc,
+                              const int32_t *__restrict__ ear, int64_t npairs, const int32_t *__restrict__ qs,
+                              const int32_t *__restrict__ qt, int32_t *__restrict__ out) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < npairs; i += (int64_t)gridDim.x * blockDim.x) {
+    const int32_t s = qs[i], t = qt[i];
+    const VDesc a = desc[s], b = desc[t];
+    const int32_t *Dp = D + (int64_t)a.p * ldd, *Dq = D + (int64_t)a.q * ldd;
+    // R[e,t] for e in {p_s, q_s} (2-term), then the 4-term rule
+    const int32_t rp = min(__viaddmin_s32(Dp[b.q], b.cq, Dp[b.p] + b.cp), INF);
+    const int32_t rq = min(__viaddmin_s32(Dq[b.q], b.cq, Dq[b.p] + b.cp), INF);
+    int32_t v = min(__viaddmin_s32(a.cq, rq, a.cp + rp), INF);
+    const int32_t es = ear[s];
+    if (es >= 0 && es == ear[t]) v = min(v, abs(a.cp - b.cp));   // same chain (C8/C9)
+    out[i] = v;
+  }
+}
+
+
 bool g_attr_set = false;
 
 }  // namespace
@@ -211,6 +237,15 @@ ear_status_t expand(const ear_plan_s *plan, const int32_t *D, int64_t ldd, int32
                                       row_end, out, ldo);
     prof_end(ss, st, 0);
   }
+  EAR_CUDA_TRY(cudaGetLastError());
+  return EAR_OK;
+}
+
+ear_status_t query_pairs(const ear_plan_s *plan, const int32_t *D, int64_t ldd, int64_t npairs, const int32_t *qs,
+                         const int32_t *qt, int32_t *out, cudaStream_t st) {
+  if (npairs <= 0) return EAR_OK;
+  const int grid = (int)std::min<int64_t>(ceil_div(npairs, 256), 148 * 16);
+  EAR_LAUNCH(k_query_pairs, grid, 256, 0, st)(D, ldd, plan->desc, plan->ear, npairs, qs, qt, out);
   EAR_CUDA_TRY(cudaGetLastError());
   return EAR_OK;
 }

@@ -20,6 +20,7 @@
 
 #include <algorithm>
 #include <cmath>
+#include <cstdlib>
 #include <vector>
 
 #include "common.cuh"
@@ -28,9 +29,6 @@ namespace ear {
 namespace {
 
 constexpr int NT = 256;
-constexpr int KC = 32;                       // k-chunk depth
-constexpr int NCHUNK = TILE / KC;            // 4
-constexpr int SM_CHUNK = KC * TILE;          // ints per operand chunk (16 KB)
 
 __global__ void k_init_D(int32_t *D, int64_t ldd, int32_t Np, int32_t row0, int32_t rows) {
   int64_t total = (int64_t)rows * (Np / 4);
@@ -118,8 +116,19 @@ __global__ void __launch_bounds__(NT, 1) k_fw_phase1(int32_t *T, int64_t ldt) {
 // Thread 0 doubles as the TMA producer.  The C tile lives in registers (8x8 per thread).
 enum { MODE_PIVOT_ROW = 0, MODE_UPPER = 1, MODE_ROWS = 2 };
 
-constexpr int STAGES = 3;
-constexpr int FW_SMEM = STAGES * 2 * SM_CHUNK * 4 + 2 * STAGES * 8;
+// Kernel variant: k-chunk depth, ring depth, C tile prefetched by TMA into shared memory (else
+// loaded straight into registers), CTAs per SM.
+template <int KC_, int ST_, bool CPF_, int MINB_>
+struct FwCfg {
+  static constexpr int KC = KC_;                       // k-chunk depth
+  static constexpr int NCHUNK = TILE / KC_;
+  static constexpr int SM_CHUNK = KC_ * TILE;          // ints per operand chunk
+  static constexpr int STAGES = ST_;
+  static constexpr bool CPF = CPF_;
+  static constexpr int MINB = MINB_;
+  static constexpr int SM_CTILE = CPF_ ? TILE * TILE : 0;
+  static constexpr int SMEM = (STAGES * 2 * SM_CHUNK + SM_CTILE) * 4 + (2 * STAGES + 2) * 8;
+};
 
 struct TileJob {
   int32_t *C;        // matrix holding the C tiles (local rows), leading dimension ldc
@@ -198,61 +207,100 @@ __device__ __forceinline__ void decode_tile(const TileJob &J, int64_t idx, int &
   tj = cidx < k ? cidx : cidx + 1;
 }
 
-__global__ void __launch_bounds__(NT, 2) k_fw_tiles(const __grid_constant__ CUtensorMap tmP, const TileJob J) {
+template <class CF>
+__global__ void __launch_bounds__(NT, CF::MINB) k_fw_tiles(const __grid_constant__ CUtensorMap tmP,
+                                                         const __grid_constant__ CUtensorMap tmC, const TileJob J) {
+  constexpr int KC = CF::KC, NCHUNK = CF::NCHUNK, SM_CHUNK = CF::SM_CHUNK, STAGES = CF::STAGES;
   extern __shared__ __align__(128) int32_t smem[];
-  int32_t *sA = smem;                                   // [STAGES][KC][TILE]   A^T chunks
-  int32_t *sB = smem + STAGES * SM_CHUNK;               // [STAGES][KC][TILE]   B chunks
-  uint64_t *full = reinterpret_cast<uint64_t *>(smem + 2 * STAGES * SM_CHUNK);
+  int32_t *sC = smem;                                   // [TILE][TILE]        next C tile (CPF only)
+  int32_t *sA = smem + CF::SM_CTILE;                    // [STAGES][KC][TILE]  A^T chunks
+  int32_t *sB = sA + STAGES * SM_CHUNK;                 // [STAGES][KC][TILE]  B chunks
+  uint64_t *full = reinterpret_cast<uint64_t *>(sB + STAGES * SM_CHUNK);
   uint64_t *empty = full + STAGES;
+  uint64_t *cfull = empty + STAGES;
+  uint64_t *cempty = cfull + 1;
   const int tid = threadIdx.x, lane = tid & 31;
   const int tx = tid & 15, ty = tid >> 4;
 
-  if (tid == 0) {
-    for (int s = 0; s < STAGES; ++s) {
-      mbar_init(&full[s], 1);
-      mbar_init(&empty[s], NT / 32);
-    }
-    asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
-    asm volatile("prefetch.tensormap [%0];\n" ::"l"(reinterpret_cast<uint64_t>(&tmP)) : "memory");
-  }
-  __syncthreads();
-
-  const int64_t my_tiles = J.ntiles > (int64_t)blockIdx.x ? (J.ntiles - 1 - blockIdx.x) / gridDim.x + 1 : 0;
-  const int64_t total_chunks = my_tiles * NCHUNK;
-  int64_t issued = 0;   // producer state (thread 0 only)
-  auto produce = [&](int64_t upto) {
+  const int my_tiles = J.ntiles > (int64_t)blockIdx.x ? (int)((J.ntiles - 1 - blockIdx.x) / gridDim.x + 1) : 0;
+  const int total_chunks = my_tiles * NCHUNK;
+  int issued = 0;   // producer state (thread 0 only)
+  auto tile_of = [&](int it, int &ti, int &tj) { decode_tile(J, blockIdx.x + (int64_t)it * gridDim.x, ti, tj); };
+  auto produce = [&](int upto) {
     while (issued < upto) {
-      const int st = (int)(issued % STAGES);
+      const int st = issued % STAGES;
       if (issued >= STAGES) mbar_wait(&empty[st], (uint32_t)((issued / STAGES - 1) & 1));
       int pti, ptj;
-      decode_tile(J, blockIdx.x + (issued / NCHUNK) * gridDim.x, pti, ptj);
-      const int row = J.p_row0 + (int)(issued % NCHUNK) * KC;
+      tile_of(issued / NCHUNK, pti, ptj);
+      const int row = J.p_row0 + (issued % NCHUNK) * KC;
       mbar_arrive_tx(&full[st], 2 * SM_CHUNK * 4);
       tma_load_2d(sA + st * SM_CHUNK, &tmP, pti * TILE, row, &full[st]);
       tma_load_2d(sB + st * SM_CHUNK, &tmP, ptj * TILE, row, &full[st]);
       ++issued;
     }
   };
-  if (tid == 0) produce(total_chunks < STAGES ? total_chunks : STAGES);
+  auto load_c = [&](int it) {
+    int cti, ctj;
+    tile_of(it, cti, ctj);
+    mbar_arrive_tx(cfull, TILE * TILE * 4);
+    tma_load_2d(sC, &tmC, ctj * TILE, (cti - J.ti0) * TILE, cfull);
+  };
 
-  int64_t g = 0;   // chunk counter (all threads)
-  for (int64_t it = 0; it < my_tiles; ++it) {
+  if (tid == 0) {
+    for (int s = 0; s < STAGES; ++s) {
+      mbar_init(&full[s], 1);
+      mbar_init(&empty[s], NT / 32);
+    }
+    mbar_init(cfull, 1);
+    mbar_init(cempty, NT / 32);
+    asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
+    asm volatile("prefetch.tensormap [%0];\n" ::"l"(reinterpret_cast<uint64_t>(&tmP)) : "memory");
+    if (CF::CPF) asm volatile("prefetch.tensormap [%0];\n" ::"l"(reinterpret_cast<uint64_t>(&tmC)) : "memory");
+  }
+  __syncthreads();
+  if (tid == 0 && my_tiles > 0) {
+    if (CF::CPF) load_c(0);
+    produce(total_chunks < STAGES ? total_chunks : STAGES);
+  }
+
+  int g = 0;   // chunk counter (all threads)
+  for (int it = 0; it < my_tiles; ++it) {
     int ti, tj;
-    decode_tile(J, blockIdx.x + it * gridDim.x, ti, tj);
-    int32_t *Ct = J.C + (int64_t)(ti - J.ti0) * TILE * J.ldc + (int64_t)tj * TILE;
+    tile_of(it, ti, tj);
     int32_t c[8][8];
+    if (CF::CPF) {   // C tile prefetched into shared memory by TMA during the previous tile
+      mbar_wait(cfull, (uint32_t)(it & 1));
 #pragma unroll
-    for (int r = 0; r < 8; ++r) {
-      const int i = (r < 4 ? 0 : 64) + ty * 4 + (r & 3);
-      const int4 lo = *reinterpret_cast<const int4 *>(Ct + (int64_t)i * J.ldc + tx * 4);
-      const int4 hi = *reinterpret_cast<const int4 *>(Ct + (int64_t)i * J.ldc + 64 + tx * 4);
-      c[r][0] = lo.x; c[r][1] = lo.y; c[r][2] = lo.z; c[r][3] = lo.w;
-      c[r][4] = hi.x; c[r][5] = hi.y; c[r][6] = hi.z; c[r][7] = hi.w;
+      for (int r = 0; r < 8; ++r) {
+        const int i = (r < 4 ? 0 : 64) + ty * 4 + (r & 3);
+        const int4 lo = *reinterpret_cast<const int4 *>(sC + i * TILE + tx * 4);
+        const int4 hi = *reinterpret_cast<const int4 *>(sC + i * TILE + 64 + tx * 4);
+        c[r][0] = lo.x; c[r][1] = lo.y; c[r][2] = lo.z; c[r][3] = lo.w;
+        c[r][4] = hi.x; c[r][5] = hi.y; c[r][6] = hi.z; c[r][7] = hi.w;
+      }
+      __syncwarp();
+      if (lane == 0) mbar_arrive(cempty);
+    } else {         // C tile straight from global memory into registers
+      const int32_t *Ct = J.C + (int64_t)(ti - J.ti0) * TILE * J.ldc + (int64_t)tj * TILE;
+#pragma unroll
+      for (int r = 0; r < 8; ++r) {
+        const int i = (r < 4 ? 0 : 64) + ty * 4 + (r & 3);
+        const int4 lo = *reinterpret_cast<const int4 *>(Ct + (int64_t)i * J.ldc + tx * 4);
+        const int4 hi = *reinterpret_cast<const int4 *>(Ct + (int64_t)i * J.ldc + 64 + tx * 4);
+        c[r][0] = lo.x; c[r][1] = lo.y; c[r][2] = lo.z; c[r][3] = lo.w;
+        c[r][4] = hi.x; c[r][5] = hi.y; c[r][6] = hi.z; c[r][7] = hi.w;
+      }
     }
 #pragma unroll 1
     for (int kc = 0; kc < NCHUNK; ++kc, ++g) {
-      if (tid == 0) produce(g + STAGES < total_chunks ? g + STAGES : total_chunks);
-      const int st = (int)(g % STAGES);
+      if (tid == 0) {
+        produce(g + STAGES < total_chunks ? g + STAGES : total_chunks);
+        if (CF::CPF && kc == 1 && it + 1 < my_tiles) {   // every warp has read this tile's C by now
+          mbar_wait(cempty, (uint32_t)(it & 1));
+          load_c(it + 1);
+        }
+      }
+      const int st = g % STAGES;
       mbar_wait(&full[st], (uint32_t)((g / STAGES) & 1));
       const int32_t *a_s = sA + st * SM_CHUNK;
       const int32_t *b_s = sB + st * SM_CHUNK;
@@ -273,6 +321,7 @@ __global__ void __launch_bounds__(NT, 2) k_fw_tiles(const __grid_constant__ CUte
       if (lane == 0) mbar_arrive(&empty[st]);
     }
     // epilogue: tile, and (single GPU, off-diagonal) its transposed mirror
+    int32_t *Ct = J.C + (int64_t)(ti - J.ti0) * TILE * J.ldc + (int64_t)tj * TILE;
 #pragma unroll
     for (int r = 0; r < 8; ++r) {
       const int i = (r < 4 ? 0 : 64) + ty * 4 + (r & 3);
@@ -308,12 +357,11 @@ __global__ void k_col_tiles_from_pivot(int32_t *C, int64_t ldc, const int32_t *P
     C[(int64_t)(tile * TILE + bx * 32 + yy) * ldc + (int64_t)k * TILE + by * 32 + lx] = t[lx][yy];
 }
 
-bool g_smem_set = false;
 int g_num_sms = 0;
 PFN_cuTensorMapEncodeTiled_v12000 g_encode = nullptr;
 
-// 2-D int32 tensor map over rows x cols (leading dimension ld elements) with a 32 x 128 box
-ear_status_t make_map(CUtensorMap *map, const int32_t *base, int64_t rows, int64_t cols, int64_t ld) {
+// 2-D int32 tensor map over rows x cols (leading dimension ld elements) with a box_rows x 128 box
+ear_status_t make_map(CUtensorMap *map, const int32_t *base, int64_t rows, int64_t cols, int64_t ld, int box_rows) {
   if (!g_encode) {
     cudaDriverEntryPointQueryResult q;
     void *fn = nullptr;
@@ -326,7 +374,7 @@ ear_status_t make_map(CUtensorMap *map, const int32_t *base, int64_t rows, int64
   }
   cuuint64_t dims[2] = {(cuuint64_t)cols, (cuuint64_t)rows};
   cuuint64_t strides[1] = {(cuuint64_t)ld * sizeof(int32_t)};
-  cuuint32_t box[2] = {(cuuint32_t)TILE, (cuuint32_t)KC};
+  cuuint32_t box[2] = {(cuuint32_t)TILE, (cuuint32_t)box_rows};
   cuuint32_t estr[2] = {1, 1};
   CUresult r = g_encode(map, CU_TENSOR_MAP_DATA_TYPE_INT32, 2, (void *)base, dims, strides, box, estr,
                         CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
@@ -339,19 +387,71 @@ ear_status_t make_map(CUtensorMap *map, const int32_t *base, int64_t rows, int64
   return EAR_OK;
 }
 
-ear_status_t launch_tiles(const CUtensorMap &map, TileJob J, int64_t nblocks, cudaStream_t st) {
-  if (!g_smem_set) {
-    EAR_CUDA_TRY(cudaFuncSetAttribute(k_fw_tiles, cudaFuncAttributeMaxDynamicSharedMemorySize, FW_SMEM));
+// ---- kernel variants (EAR_FW_VARIANT selects one for experiments; 0 is the default)
+using V0 = FwCfg<32, 3, false, 2>;   // 96 KB ring, C via LDG, 2 CTAs/SM
+using V1 = FwCfg<16, 3, true, 2>;    // 48 KB ring + 64 KB C prefetch, 2 CTAs/SM
+using V2 = FwCfg<16, 4, false, 2>;   // 64 KB ring, C via LDG, 2 CTAs/SM
+using V3 = FwCfg<32, 2, true, 1>;    // 64 KB ring + 64 KB C prefetch, 1 CTA/SM
+using V4 = FwCfg<64, 2, false, 1>;   // 128 KB ring, C via LDG, 1 CTA/SM
+using V5 = FwCfg<64, 2, true, 1>;    // 128 KB ring + 64 KB C prefetch, 1 CTA/SM
+using V6 = FwCfg<32, 4, true, 1>;    // 128 KB ring (4 stages) + 64 KB C prefetch, 1 CTA/SM
+int g_variant = -1;
+
+int fw_variant() {
+  if (g_variant < 0) {
+    const char *e = getenv("EAR_FW_VARIANT");
+    g_variant = e ? atoi(e) : 0;
+    if (g_variant < 0 || g_variant > 6) g_variant = 0;
+  }
+  return g_variant;
+}
+
+int fw_kc() {
+  switch (fw_variant()) {
+    case 1: return V1::KC;
+    case 2: return V2::KC;
+    case 3: return V3::KC;
+    case 4: return V4::KC;
+    case 5: return V5::KC;
+    case 6: return V6::KC;
+    default: return V0::KC;
+  }
+}
+
+template <class CF>
+ear_status_t launch_variant(const CUtensorMap &map, const CUtensorMap &cmap, const TileJob &J, int64_t nblocks,
+                            cudaStream_t st) {
+  static bool attr = false;
+  if (!attr) {
+    EAR_CUDA_TRY(cudaFuncSetAttribute(k_fw_tiles<CF>, cudaFuncAttributeMaxDynamicSharedMemorySize, CF::SMEM));
+    attr = true;
+  }
+  int per_sm = 0;
+  EAR_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_fw_tiles<CF>, NT, CF::SMEM));
+  if (per_sm < 1) per_sm = 1;
+  const int64_t grid = std::min<int64_t>(nblocks, (int64_t)g_num_sms * per_sm);   // persistent
+  EAR_LAUNCH(k_fw_tiles<CF>, (unsigned)grid, NT, CF::SMEM, st)(map, cmap, J);
+  return EAR_OK;
+}
+
+ear_status_t launch_tiles(const CUtensorMap &map, const CUtensorMap &cmap, TileJob J, int64_t nblocks,
+                          cudaStream_t st) {
+  if (!g_num_sms) {
     int dev = 0;
     EAR_CUDA_TRY(cudaGetDevice(&dev));
     EAR_CUDA_TRY(cudaDeviceGetAttribute(&g_num_sms, cudaDevAttrMultiProcessorCount, dev));
-    g_smem_set = true;
   }
   if (nblocks <= 0) return EAR_OK;
   J.ntiles = nblocks;
-  const int64_t grid = std::min<int64_t>(nblocks, (int64_t)g_num_sms * 2);   // persistent: 2 CTAs / SM
-  EAR_LAUNCH(k_fw_tiles, (unsigned)grid, NT, FW_SMEM, st)(map, J);
-  return EAR_OK;
+  switch (fw_variant()) {
+    case 1: return launch_variant<V1>(map, cmap, J, nblocks, st);
+    case 2: return launch_variant<V2>(map, cmap, J, nblocks, st);
+    case 3: return launch_variant<V3>(map, cmap, J, nblocks, st);
+    case 4: return launch_variant<V4>(map, cmap, J, nblocks, st);
+    case 5: return launch_variant<V5>(map, cmap, J, nblocks, st);
+    case 6: return launch_variant<V6>(map, cmap, J, nblocks, st);
+    default: return launch_variant<V0>(map, cmap, J, nblocks, st);
+  }
 }
 
 }  // namespace
@@ -375,8 +475,9 @@ ear_status_t fw_init_D(const ear_plan_s *plan, int32_t *D, int64_t ldd, int32_t 
 ear_status_t fw_single(int32_t *D, int64_t ldd, int32_t Np, cudaStream_t st) {
   const int nt = Np / TILE;
   const double tile_ops = (double)TILE * TILE * TILE;
-  CUtensorMap map;
-  EAR_TRY(make_map(&map, D, Np, Np, ldd));
+  CUtensorMap map, cmap;
+  EAR_TRY(make_map(&map, D, Np, Np, ldd, fw_kc()));
+  EAR_TRY(make_map(&cmap, D, Np, Np, ldd, TILE));
   for (int k = 0; k < nt; ++k) {
     int32_t *Pk = D + (int64_t)k * TILE * ldd;            // pivot row block
     int s1 = prof_begin(PK_FW_P1, st);
@@ -384,12 +485,12 @@ ear_status_t fw_single(int32_t *D, int64_t ldd, int32_t Np, cudaStream_t st) {
     prof_end(s1, st, tile_ops);
     TileJob J{D, ldd, k * TILE, k, nt, 0, nt, MODE_PIVOT_ROW, 1, 0};
     int s2 = prof_begin(PK_FW_P2, st);
-    EAR_TRY(launch_tiles(map, J, nt - 1, st));
+    EAR_TRY(launch_tiles(map, cmap, J, nt - 1, st));
     prof_end(s2, st, (nt - 1) * tile_ops);
     J.mode = MODE_UPPER;
     const int64_t nup = (int64_t)(nt - 1) * nt / 2;
     int s3 = prof_begin(PK_FW_P3, st);
-    EAR_TRY(launch_tiles(map, J, nup, st));
+    EAR_TRY(launch_tiles(map, cmap, J, nup, st));
     prof_end(s3, st, nup * tile_ops);
   }
   EAR_CUDA_TRY(cudaGetLastError());
@@ -406,15 +507,16 @@ struct ShardCtx {
   int64_t ldd;
   int32_t Np, nt, P, rank, nti, ti0;
   int32_t *prow;    // 128 x Np pivot row block (leading dimension Np)
-  CUtensorMap map_blk, map_prow;
+  CUtensorMap map_blk, map_prow, map_c;
 };
 
 static ear_status_t shard_ctx(ShardCtx *c, int32_t *Dblk, int64_t ldd, int32_t Np, int32_t P, int32_t rank,
                               int32_t *prow) {
   c->Dblk = Dblk; c->ldd = ldd; c->Np = Np; c->nt = Np / TILE; c->P = P; c->rank = rank;
   c->nti = c->nt / P; c->ti0 = rank * c->nti; c->prow = prow;
-  EAR_TRY(make_map(&c->map_blk, Dblk, (int64_t)c->nti * TILE, Np, ldd));
-  EAR_TRY(make_map(&c->map_prow, prow, TILE, Np, Np));
+  EAR_TRY(make_map(&c->map_blk, Dblk, (int64_t)c->nti * TILE, Np, ldd, fw_kc()));
+  EAR_TRY(make_map(&c->map_c, Dblk, (int64_t)c->nti * TILE, Np, ldd, TILE));
+  EAR_TRY(make_map(&c->map_prow, prow, TILE, Np, Np, fw_kc()));
   return EAR_OK;
 }
 
@@ -425,9 +527,10 @@ static ear_status_t shard_owner_step(const ShardCtx &c, int k, cudaStream_t st) 
   EAR_LAUNCH(k_fw_phase1, 1, NT, 0, st)(Pk + (int64_t)k * TILE, c.ldd);
   prof_end(s1, st, tile_ops);
   // pivot-row tiles; C rows are the pivot rows themselves (ti0 = k: local row offset 0)
-  TileJob J{Pk, c.ldd, (k - c.ti0) * TILE, k, c.nt, k, 1, MODE_PIVOT_ROW, 0, 0};
+  // pivot-row tiles (ti = k inside this rank's block)
+  TileJob J{c.Dblk, c.ldd, (k - c.ti0) * TILE, k, c.nt, c.ti0, c.nti, MODE_PIVOT_ROW, 0, 0};
   int s2 = prof_begin(PK_FW_P2, st);
-  EAR_TRY(launch_tiles(c.map_blk, J, c.nt - 1, st));
+  EAR_TRY(launch_tiles(c.map_blk, c.map_c, J, c.nt - 1, st));
   prof_end(s2, st, (c.nt - 1) * tile_ops);
   EAR_CUDA_TRY(cudaMemcpy2DAsync(c.prow, sizeof(int32_t) * c.Np, Pk, sizeof(int32_t) * c.ldd,
                                  sizeof(int32_t) * c.Np, TILE, cudaMemcpyDeviceToDevice, st));
@@ -442,7 +545,7 @@ static ear_status_t shard_update_step(const ShardCtx &c, int k, cudaStream_t st)
   const int rows_here = (owner == c.rank) ? c.nti - 1 : c.nti;
   TileJob J{c.Dblk, c.ldd, 0, k, c.nt, c.ti0, c.nti, MODE_ROWS, 0, 0};
   int s3 = prof_begin(PK_FW_P3, st);
-  EAR_TRY(launch_tiles(c.map_prow, J, (int64_t)rows_here * (c.nt - 1), st));
+  EAR_TRY(launch_tiles(c.map_prow, c.map_c, J, (int64_t)rows_here * (c.nt - 1), st));
   prof_end(s3, st, (double)rows_here * (c.nt - 1) * tile_ops);
   return EAR_OK;
 }

@@ -63,6 +63,7 @@ SIGNATURES = {
     "apsp_reduced_emulated": (_I32, [_P, _I32, _P, _I64, _P]),
     "ear_gather_reduced": (_I32, [_P, _P, _I64, _P, _I64, _P, _P]),
     "expand_ears": (_I32, [_P, _P, _I64, _I32, _I32, _P, _I64, _P]),
+    "ear_query_pairs": (_I32, [_P, _P, _I64, _I64, _P, _P, _P, _P]),
     "apsp_full": (_I32, [_I32, _I64, _P, _P, _P, _U32, _I32, _I32, _P, _I64, _P, _P]),
     "apsp_full_host": (_I32, [_I32, _I64, _P, _P, _P, _U32, _I32, _I32, _P, _I64, _P, _P]),
     "ear_row_block": (None, [_I32, _I32, _I32, ctypes.POINTER(_I32), ctypes.POINTER(_I32)]),
@@ -259,6 +260,17 @@ def expand_ears(plan: Plan, D_full: torch.Tensor, row_begin: int, row_end: int, 
         raise EarError("out must be an int32 CUDA tensor with unit column stride")
     _check(lib().expand_ears(plan.handle, D_full.data_ptr(), D_full.stride(0), row_begin, row_end, out.data_ptr(),
                              out.stride(0), _stream(stream)), "expand_ears")
+    return out
+
+
+def query_pairs(plan: Plan, D_full: torch.Tensor, s: torch.Tensor, t: torch.Tensor,
+                out: torch.Tensor | None = None, stream=None) -> torch.Tensor:
+    """Compact/query mode: S[s[i], t[i]] from D and the plan's descriptors (no N x N matrix)."""
+    s, t = _dev_i32(s, "s"), _dev_i32(t, "t")
+    if out is None:
+        out = torch.empty(s.numel(), dtype=torch.int32, device="cuda")
+    _check(lib().ear_query_pairs(plan.handle, _dev_i32(D_full, "D_full").data_ptr(), D_full.stride(0), s.numel(),
+                                 s.data_ptr(), t.data_ptr(), out.data_ptr(), _stream(stream)), "ear_query_pairs")
     return out
 
 

@@ -270,3 +270,35 @@ def test_sharded_schedule_emulated_corner(pkg, seed):
     full = pkg.expand_ears(plan, DP, 0, g.n).cpu().numpy()
     assert_exact(full, oracle.apsp(g.n, g.src, g.dst, g.w), f"emulated P=3 seed {seed}")
     assert nr > 0
+
+
+# ------------------------------------------------------------------------------ NEXT 1: query mode
+@pytest.mark.parametrize("name", ["corner", "cfg2"])
+def test_query_pairs(pkg, name):
+    g = gg.corner_cases(31, n_target=500) if name == "corner" else gg.config("cfg2")
+    plan = pkg.ear_decompose(g.n, dev(g.src), dev(g.dst), dev(g.w))
+    D = pkg.alloc_D(plan)
+    pkg.apsp_reduced(plan, D)
+    rng = np.random.default_rng(7)
+    rows = rng.choice(g.n, min(g.n, 40), replace=False)
+    ref = oracle.apsp_rows(g.n, g.src, g.dst, g.w, rows)
+    s = np.repeat(rows, g.n).astype(np.int32)
+    t = np.tile(np.arange(g.n), len(rows)).astype(np.int32)
+    got = pkg.query_pairs(plan, D, dev(s), dev(t)).cpu().numpy().reshape(len(rows), g.n)
+    assert_exact(got, ref, f"query pairs {name}")
+
+
+def test_query_pairs_cfg4_without_full_matrix(pkg):
+    """Compact mode at full size: D (3.6 GB) + descriptors, random pairs vs oracle rows."""
+    g = gg.config("cfg4")
+    plan = pkg.ear_decompose(g.n, dev(g.src), dev(g.dst), dev(g.w))
+    D = pkg.alloc_D(plan)
+    pkg.apsp_reduced(plan, D)
+    rng = np.random.default_rng(11)
+    rows = rng.choice(g.n, 16, replace=False)
+    ref = oracle.apsp_rows(g.n, g.src, g.dst, g.w, rows)
+    cols = rng.choice(g.n, 5000, replace=False)
+    s = np.repeat(rows, len(cols)).astype(np.int32)
+    t = np.tile(cols, len(rows)).astype(np.int32)
+    got = pkg.query_pairs(plan, D, dev(s), dev(t)).cpu().numpy().reshape(len(rows), len(cols))
+    assert_exact(got, ref[:, cols], "cfg4 query pairs")
