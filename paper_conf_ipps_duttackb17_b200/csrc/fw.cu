@@ -20,7 +20,6 @@
 
 #include <algorithm>
 #include <cmath>
-#include <cstdlib>
 #include <vector>
 
 #include "common.cuh"
@@ -116,18 +115,16 @@ __global__ void __launch_bounds__(NT, 1) k_fw_phase1(int32_t *T, int64_t ldt) {
 // Thread 0 doubles as the TMA producer.  The C tile lives in registers (8x8 per thread).
 enum { MODE_PIVOT_ROW = 0, MODE_UPPER = 1, MODE_ROWS = 2 };
 
-// Kernel variant: k-chunk depth, ring depth, C tile prefetched by TMA into shared memory (else
-// loaded straight into registers), CTAs per SM.
-template <int KC_, int ST_, bool CPF_, int MINB_>
+// Tile-kernel configuration: k-chunk depth, TMA ring depth, CTAs per SM, kk-loop unroll.
+template <int KC_, int ST_, int MINB_, int UNR_>
 struct FwCfg {
-  static constexpr int KC = KC_;                       // k-chunk depth
+  static constexpr int KC = KC_;
   static constexpr int NCHUNK = TILE / KC_;
   static constexpr int SM_CHUNK = KC_ * TILE;          // ints per operand chunk
   static constexpr int STAGES = ST_;
-  static constexpr bool CPF = CPF_;
   static constexpr int MINB = MINB_;
-  static constexpr int SM_CTILE = CPF_ ? TILE * TILE : 0;
-  static constexpr int SMEM = (STAGES * 2 * SM_CHUNK + SM_CTILE) * 4 + (2 * STAGES + 2) * 8;
+  static constexpr int UNR = UNR_;
+  static constexpr int SMEM = STAGES * 2 * SM_CHUNK * 4 + 2 * STAGES * 8;
 };
 
 struct TileJob {
@@ -208,17 +205,13 @@ __device__ __forceinline__ void decode_tile(const TileJob &J, int64_t idx, int &
 }
 
 template <class CF>
-__global__ void __launch_bounds__(NT, CF::MINB) k_fw_tiles(const __grid_constant__ CUtensorMap tmP,
-                                                         const __grid_constant__ CUtensorMap tmC, const TileJob J) {
+__global__ void __launch_bounds__(NT, CF::MINB) k_fw_tiles(const __grid_constant__ CUtensorMap tmP, const TileJob J) {
   constexpr int KC = CF::KC, NCHUNK = CF::NCHUNK, SM_CHUNK = CF::SM_CHUNK, STAGES = CF::STAGES;
   extern __shared__ __align__(128) int32_t smem[];
-  int32_t *sC = smem;                                   // [TILE][TILE]        next C tile (CPF only)
-  int32_t *sA = smem + CF::SM_CTILE;                    // [STAGES][KC][TILE]  A^T chunks
+  int32_t *sA = smem;                                   // [STAGES][KC][TILE]  A^T chunks
   int32_t *sB = sA + STAGES * SM_CHUNK;                 // [STAGES][KC][TILE]  B chunks
   uint64_t *full = reinterpret_cast<uint64_t *>(sB + STAGES * SM_CHUNK);
   uint64_t *empty = full + STAGES;
-  uint64_t *cfull = empty + STAGES;
-  uint64_t *cempty = cfull + 1;
   const int tid = threadIdx.x, lane = tid & 31;
   const int tx = tid & 15, ty = tid >> 4;
 
@@ -239,72 +232,41 @@ __global__ void __launch_bounds__(NT, CF::MINB) k_fw_tiles(const __grid_constant
       ++issued;
     }
   };
-  auto load_c = [&](int it) {
-    int cti, ctj;
-    tile_of(it, cti, ctj);
-    mbar_arrive_tx(cfull, TILE * TILE * 4);
-    tma_load_2d(sC, &tmC, ctj * TILE, (cti - J.ti0) * TILE, cfull);
-  };
 
   if (tid == 0) {
     for (int s = 0; s < STAGES; ++s) {
       mbar_init(&full[s], 1);
       mbar_init(&empty[s], NT / 32);
     }
-    mbar_init(cfull, 1);
-    mbar_init(cempty, NT / 32);
     asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
     asm volatile("prefetch.tensormap [%0];\n" ::"l"(reinterpret_cast<uint64_t>(&tmP)) : "memory");
-    if (CF::CPF) asm volatile("prefetch.tensormap [%0];\n" ::"l"(reinterpret_cast<uint64_t>(&tmC)) : "memory");
   }
   __syncthreads();
-  if (tid == 0 && my_tiles > 0) {
-    if (CF::CPF) load_c(0);
-    produce(total_chunks < STAGES ? total_chunks : STAGES);
-  }
+  if (tid == 0 && my_tiles > 0) produce(total_chunks < STAGES ? total_chunks : STAGES);
 
   int g = 0;   // chunk counter (all threads)
   for (int it = 0; it < my_tiles; ++it) {
     int ti, tj;
     tile_of(it, ti, tj);
     int32_t c[8][8];
-    if (CF::CPF) {   // C tile prefetched into shared memory by TMA during the previous tile
-      mbar_wait(cfull, (uint32_t)(it & 1));
+    // C tile straight from global memory into registers (its latency overlaps the in-flight TMA chunks)
+    int32_t *Ct = J.C + (int64_t)(ti - J.ti0) * TILE * J.ldc + (int64_t)tj * TILE;
 #pragma unroll
-      for (int r = 0; r < 8; ++r) {
-        const int i = (r < 4 ? 0 : 64) + ty * 4 + (r & 3);
-        const int4 lo = *reinterpret_cast<const int4 *>(sC + i * TILE + tx * 4);
-        const int4 hi = *reinterpret_cast<const int4 *>(sC + i * TILE + 64 + tx * 4);
-        c[r][0] = lo.x; c[r][1] = lo.y; c[r][2] = lo.z; c[r][3] = lo.w;
-        c[r][4] = hi.x; c[r][5] = hi.y; c[r][6] = hi.z; c[r][7] = hi.w;
-      }
-      __syncwarp();
-      if (lane == 0) mbar_arrive(cempty);
-    } else {         // C tile straight from global memory into registers
-      const int32_t *Ct = J.C + (int64_t)(ti - J.ti0) * TILE * J.ldc + (int64_t)tj * TILE;
-#pragma unroll
-      for (int r = 0; r < 8; ++r) {
-        const int i = (r < 4 ? 0 : 64) + ty * 4 + (r & 3);
-        const int4 lo = *reinterpret_cast<const int4 *>(Ct + (int64_t)i * J.ldc + tx * 4);
-        const int4 hi = *reinterpret_cast<const int4 *>(Ct + (int64_t)i * J.ldc + 64 + tx * 4);
-        c[r][0] = lo.x; c[r][1] = lo.y; c[r][2] = lo.z; c[r][3] = lo.w;
-        c[r][4] = hi.x; c[r][5] = hi.y; c[r][6] = hi.z; c[r][7] = hi.w;
-      }
+    for (int r = 0; r < 8; ++r) {
+      const int i = (r < 4 ? 0 : 64) + ty * 4 + (r & 3);
+      const int4 lo = *reinterpret_cast<const int4 *>(Ct + (int64_t)i * J.ldc + tx * 4);
+      const int4 hi = *reinterpret_cast<const int4 *>(Ct + (int64_t)i * J.ldc + 64 + tx * 4);
+      c[r][0] = lo.x; c[r][1] = lo.y; c[r][2] = lo.z; c[r][3] = lo.w;
+      c[r][4] = hi.x; c[r][5] = hi.y; c[r][6] = hi.z; c[r][7] = hi.w;
     }
 #pragma unroll 1
     for (int kc = 0; kc < NCHUNK; ++kc, ++g) {
-      if (tid == 0) {
-        produce(g + STAGES < total_chunks ? g + STAGES : total_chunks);
-        if (CF::CPF && kc == 1 && it + 1 < my_tiles) {   // every warp has read this tile's C by now
-          mbar_wait(cempty, (uint32_t)(it & 1));
-          load_c(it + 1);
-        }
-      }
+      if (tid == 0) produce(g + STAGES < total_chunks ? g + STAGES : total_chunks);
       const int st = g % STAGES;
       mbar_wait(&full[st], (uint32_t)((g / STAGES) & 1));
       const int32_t *a_s = sA + st * SM_CHUNK;
       const int32_t *b_s = sB + st * SM_CHUNK;
-#pragma unroll 4
+#pragma unroll CF::UNR
       for (int kk = 0; kk < KC; ++kk) {
         const int4 alo = *reinterpret_cast<const int4 *>(a_s + kk * TILE + ty * 4);
         const int4 ahi = *reinterpret_cast<const int4 *>(a_s + kk * TILE + 64 + ty * 4);
@@ -321,7 +283,6 @@ __global__ void __launch_bounds__(NT, CF::MINB) k_fw_tiles(const __grid_constant
       if (lane == 0) mbar_arrive(&empty[st]);
     }
     // epilogue: tile, and (single GPU, off-diagonal) its transposed mirror
-    int32_t *Ct = J.C + (int64_t)(ti - J.ti0) * TILE * J.ldc + (int64_t)tj * TILE;
 #pragma unroll
     for (int r = 0; r < 8; ++r) {
       const int i = (r < 4 ? 0 : 64) + ty * 4 + (r & 3);
@@ -387,40 +348,15 @@ ear_status_t make_map(CUtensorMap *map, const int32_t *base, int64_t rows, int64
   return EAR_OK;
 }
 
-// ---- kernel variants (EAR_FW_VARIANT selects one for experiments; 0 is the default)
-using V0 = FwCfg<32, 3, false, 2>;   // 96 KB ring, C via LDG, 2 CTAs/SM
-using V1 = FwCfg<16, 3, true, 2>;    // 48 KB ring + 64 KB C prefetch, 2 CTAs/SM
-using V2 = FwCfg<16, 4, false, 2>;   // 64 KB ring, C via LDG, 2 CTAs/SM
-using V3 = FwCfg<32, 2, true, 1>;    // 64 KB ring + 64 KB C prefetch, 1 CTA/SM
-using V4 = FwCfg<64, 2, false, 1>;   // 128 KB ring, C via LDG, 1 CTA/SM
-using V5 = FwCfg<64, 2, true, 1>;    // 128 KB ring + 64 KB C prefetch, 1 CTA/SM
-using V6 = FwCfg<32, 4, true, 1>;    // 128 KB ring (4 stages) + 64 KB C prefetch, 1 CTA/SM
-int g_variant = -1;
+// The tile kernel's configuration, chosen by measurement on the B200 (cfg4, phase-3 share of the
+// VIADDMNMX peak; profiles/r01_fw_variants.txt): 64-deep k-chunks, a 2-stage TMA ring (128 KB), C
+// straight into registers, one 256-thread CTA per SM (161 registers, no spills), kk unrolled 16x.
+using FwTile = FwCfg<64, 2, 1, 16>;
 
-int fw_variant() {
-  if (g_variant < 0) {
-    const char *e = getenv("EAR_FW_VARIANT");
-    g_variant = e ? atoi(e) : 0;
-    if (g_variant < 0 || g_variant > 6) g_variant = 0;
-  }
-  return g_variant;
-}
-
-int fw_kc() {
-  switch (fw_variant()) {
-    case 1: return V1::KC;
-    case 2: return V2::KC;
-    case 3: return V3::KC;
-    case 4: return V4::KC;
-    case 5: return V5::KC;
-    case 6: return V6::KC;
-    default: return V0::KC;
-  }
-}
+int fw_kc() { return FwTile::KC; }
 
 template <class CF>
-ear_status_t launch_variant(const CUtensorMap &map, const CUtensorMap &cmap, const TileJob &J, int64_t nblocks,
-                            cudaStream_t st) {
+ear_status_t launch_cfg(const CUtensorMap &map, const TileJob &J, int64_t nblocks, cudaStream_t st) {
   static bool attr = false;
   if (!attr) {
     EAR_CUDA_TRY(cudaFuncSetAttribute(k_fw_tiles<CF>, cudaFuncAttributeMaxDynamicSharedMemorySize, CF::SMEM));
@@ -430,12 +366,11 @@ ear_status_t launch_variant(const CUtensorMap &map, const CUtensorMap &cmap, con
   EAR_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_fw_tiles<CF>, NT, CF::SMEM));
   if (per_sm < 1) per_sm = 1;
   const int64_t grid = std::min<int64_t>(nblocks, (int64_t)g_num_sms * per_sm);   // persistent
-  EAR_LAUNCH(k_fw_tiles<CF>, (unsigned)grid, NT, CF::SMEM, st)(map, cmap, J);
+  EAR_LAUNCH(k_fw_tiles<CF>, (unsigned)grid, NT, CF::SMEM, st)(map, J);
   return EAR_OK;
 }
 
-ear_status_t launch_tiles(const CUtensorMap &map, const CUtensorMap &cmap, TileJob J, int64_t nblocks,
-                          cudaStream_t st) {
+ear_status_t launch_tiles(const CUtensorMap &map, TileJob J, int64_t nblocks, cudaStream_t st) {
   if (!g_num_sms) {
     int dev = 0;
     EAR_CUDA_TRY(cudaGetDevice(&dev));
@@ -443,15 +378,7 @@ ear_status_t launch_tiles(const CUtensorMap &map, const CUtensorMap &cmap, TileJ
   }
   if (nblocks <= 0) return EAR_OK;
   J.ntiles = nblocks;
-  switch (fw_variant()) {
-    case 1: return launch_variant<V1>(map, cmap, J, nblocks, st);
-    case 2: return launch_variant<V2>(map, cmap, J, nblocks, st);
-    case 3: return launch_variant<V3>(map, cmap, J, nblocks, st);
-    case 4: return launch_variant<V4>(map, cmap, J, nblocks, st);
-    case 5: return launch_variant<V5>(map, cmap, J, nblocks, st);
-    case 6: return launch_variant<V6>(map, cmap, J, nblocks, st);
-    default: return launch_variant<V0>(map, cmap, J, nblocks, st);
-  }
+  return launch_cfg<FwTile>(map, J, nblocks, st);
 }
 
 }  // namespace
@@ -475,9 +402,8 @@ ear_status_t fw_init_D(const ear_plan_s *plan, int32_t *D, int64_t ldd, int32_t 
 ear_status_t fw_single(int32_t *D, int64_t ldd, int32_t Np, cudaStream_t st) {
   const int nt = Np / TILE;
   const double tile_ops = (double)TILE * TILE * TILE;
-  CUtensorMap map, cmap;
+  CUtensorMap map;
   EAR_TRY(make_map(&map, D, Np, Np, ldd, fw_kc()));
-  EAR_TRY(make_map(&cmap, D, Np, Np, ldd, TILE));
   for (int k = 0; k < nt; ++k) {
     int32_t *Pk = D + (int64_t)k * TILE * ldd;            // pivot row block
     int s1 = prof_begin(PK_FW_P1, st);
@@ -485,12 +411,12 @@ ear_status_t fw_single(int32_t *D, int64_t ldd, int32_t Np, cudaStream_t st) {
     prof_end(s1, st, tile_ops);
     TileJob J{D, ldd, k * TILE, k, nt, 0, nt, MODE_PIVOT_ROW, 1, 0};
     int s2 = prof_begin(PK_FW_P2, st);
-    EAR_TRY(launch_tiles(map, cmap, J, nt - 1, st));
+    EAR_TRY(launch_tiles(map, J, nt - 1, st));
     prof_end(s2, st, (nt - 1) * tile_ops);
     J.mode = MODE_UPPER;
     const int64_t nup = (int64_t)(nt - 1) * nt / 2;
     int s3 = prof_begin(PK_FW_P3, st);
-    EAR_TRY(launch_tiles(map, cmap, J, nup, st));
+    EAR_TRY(launch_tiles(map, J, nup, st));
     prof_end(s3, st, nup * tile_ops);
   }
   EAR_CUDA_TRY(cudaGetLastError());
@@ -507,7 +433,7 @@ struct ShardCtx {
   int64_t ldd;
   int32_t Np, nt, P, rank, nti, ti0;
   int32_t *prow;    // 128 x Np pivot row block (leading dimension Np)
-  CUtensorMap map_blk, map_prow, map_c;
+  CUtensorMap map_blk, map_prow;
 };
 
 static ear_status_t shard_ctx(ShardCtx *c, int32_t *Dblk, int64_t ldd, int32_t Np, int32_t P, int32_t rank,
@@ -515,7 +441,6 @@ static ear_status_t shard_ctx(ShardCtx *c, int32_t *Dblk, int64_t ldd, int32_t N
   c->Dblk = Dblk; c->ldd = ldd; c->Np = Np; c->nt = Np / TILE; c->P = P; c->rank = rank;
   c->nti = c->nt / P; c->ti0 = rank * c->nti; c->prow = prow;
   EAR_TRY(make_map(&c->map_blk, Dblk, (int64_t)c->nti * TILE, Np, ldd, fw_kc()));
-  EAR_TRY(make_map(&c->map_c, Dblk, (int64_t)c->nti * TILE, Np, ldd, TILE));
   EAR_TRY(make_map(&c->map_prow, prow, TILE, Np, Np, fw_kc()));
   return EAR_OK;
 }
@@ -530,7 +455,7 @@ static ear_status_t shard_owner_step(const ShardCtx &c, int k, cudaStream_t st) 
   // pivot-row tiles (ti = k inside this rank's block)
   TileJob J{c.Dblk, c.ldd, (k - c.ti0) * TILE, k, c.nt, c.ti0, c.nti, MODE_PIVOT_ROW, 0, 0};
   int s2 = prof_begin(PK_FW_P2, st);
-  EAR_TRY(launch_tiles(c.map_blk, c.map_c, J, c.nt - 1, st));
+  EAR_TRY(launch_tiles(c.map_blk, J, c.nt - 1, st));
   prof_end(s2, st, (c.nt - 1) * tile_ops);
   EAR_CUDA_TRY(cudaMemcpy2DAsync(c.prow, sizeof(int32_t) * c.Np, Pk, sizeof(int32_t) * c.ldd,
                                  sizeof(int32_t) * c.Np, TILE, cudaMemcpyDeviceToDevice, st));
@@ -545,7 +470,7 @@ static ear_status_t shard_update_step(const ShardCtx &c, int k, cudaStream_t st)
   const int rows_here = (owner == c.rank) ? c.nti - 1 : c.nti;
   TileJob J{c.Dblk, c.ldd, 0, k, c.nt, c.ti0, c.nti, MODE_ROWS, 0, 0};
   int s3 = prof_begin(PK_FW_P3, st);
-  EAR_TRY(launch_tiles(c.map_prow, c.map_c, J, (int64_t)rows_here * (c.nt - 1), st));
+  EAR_TRY(launch_tiles(c.map_prow, J, (int64_t)rows_here * (c.nt - 1), st));
   prof_end(s3, st, (double)rows_here * (c.nt - 1) * tile_ops);
   return EAR_OK;
 }
