@@ -238,8 +238,10 @@ def run_ours(args, rank, world, local_rank):
     plan.destroy()
     stream = torch.cuda.current_stream(dev)
 
+    flags = ea.FLAG_SSSP if args.phase2 == "sssp" else 0
+
     def step():
-        ea.apsp_full(g.n, src, dst, w, out=out, row_begin=r0, row_end=r1, comm=comm, stream=stream)
+        ea.apsp_full(g.n, src, dst, w, out=out, row_begin=r0, row_end=r1, flags=flags, comm=comm, stream=stream)
 
     for _ in range(args.warmup):
         step()
@@ -291,7 +293,15 @@ def run_ours(args, rank, world, local_rank):
                        "bytes_per_launch": prof["expand_bytes"] / max(prof["expand_launches"], 1)}
     K = args.steps
     fw_ms = prof["fw_init_ms"] + prof["fw_phase1_ms"] + prof["fw_phase2_ms"] + prof["fw_phase3_ms"]
-    phases = {"decompose": prof["decompose_ms"] / K, "fw": fw_ms / K, "fw_phase1": prof["fw_phase1_ms"] / K,
+    if args.phase2 == "sssp":   # the dominant kernel is the per-source SSSP (latency / L2-atomic bound)
+        sssp_ms = prof["sssp_ms"]
+        roofline = {"bound": "latency", "kernel": "k_sssp_bf (Phase II by per-source SSSP)",
+                    "achieved": prof["sssp_arcs"] / (sssp_ms / 1e3) / 1e9 if sssp_ms > 0 else 0.0,
+                    "peak": None, "unit": "G arc-relaxations/s (one pass over G^r per source)", "frac": None,
+                    "traffic": ncu_traffic("k_sssp_bf", args.config),
+                    "avg_launch_ms": sssp_ms / max(prof["sssp_launches"], 1),
+                    "note": "label-correcting Bellman-Ford per source; no arithmetic roofline applies"}
+    phases = {"decompose": prof["decompose_ms"] / K, "fw": fw_ms / K, "sssp": prof["sssp_ms"] / K, "fw_phase1": prof["fw_phase1_ms"] / K,
               "fw_phase2": prof["fw_phase2_ms"] / K, "fw_phase3": p3_ms / K, "comm": prof["comm_ms"] / K,
               "expand": ex_ms / K, "same_chain": prof["same_chain_ms"] / K}
     fw_minplus = prof["fw_phase2_minplus"] + prof["fw_phase3_minplus"]
@@ -306,11 +316,13 @@ def run_ours(args, rank, world, local_rank):
         hw = torch.as_tensor(g.w).pin_memory()
         hout = torch.empty((rows, g.n), dtype=torch.int32, pin_memory=True)
         e2e_steps = max(1, min(args.steps, args.e2e_steps))
-        ea.apsp_full_host(g.n, hs, hd, hw, out=hout, row_begin=r0, row_end=r1, comm=comm, stream=stream)
+        ea.apsp_full_host(g.n, hs, hd, hw, out=hout, row_begin=r0, row_end=r1, flags=flags, comm=comm,
+                          stream=stream)
         barrier()
         t = time.perf_counter()
         for _ in range(e2e_steps):
-            ea.apsp_full_host(g.n, hs, hd, hw, out=hout, row_begin=r0, row_end=r1, comm=comm, stream=stream)
+            ea.apsp_full_host(g.n, hs, hd, hw, out=hout, row_begin=r0, row_end=r1, flags=flags, comm=comm,
+                              stream=stream)
         torch.cuda.synchronize()
         e2e_s = max_over_ranks(time.perf_counter() - t, world, dev)
         barrier()
@@ -336,6 +348,7 @@ def run_ours(args, rank, world, local_rank):
                            "n_chains": info.n_chains, "max_chain_len": info.max_chain_len,
                            "degree2_frac": stats["deg2_frac"], "seed": args.seed, "rows_per_rank": rows,
                            "parallelism": f"row-block x{world}" if world > 1 else "single GPU",
+                           "phase2": args.phase2,
                            "l2": "inputs larger than L2 (D %.1f GB, output %.1f GB per step)" % (
                                4.0 * info.n_reduced_padded ** 2 / 1e9, 4.0 * g.n * g.n / 1e9)},
                 "roofline": roofline, "roofline_expand": roofline_expand,
@@ -357,6 +370,8 @@ def main():
     ap.add_argument("--config", default="cfg4")
     ap.add_argument("--seed", type=int, default=0)
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
+    ap.add_argument("--phase2", choices=["fw", "sssp"], default="fw",
+                    help="Phase II algorithm: blocked FW (north star) or per-source SSSP (SURVEY 8.f NEXT 2)")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--no-cpu-baseline", action="store_true")

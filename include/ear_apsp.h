@@ -49,7 +49,9 @@ typedef enum {
 
 enum {
   EAR_FLAG_NONE = 0,
-  EAR_FLAG_NO_CONTRACT = 1 /* every vertex is a terminal: direct blocked FW on G (cfg3 baseline) */
+  EAR_FLAG_NO_CONTRACT = 1, /* every vertex is a terminal: direct blocked FW on G (cfg3 baseline) */
+  EAR_FLAG_SSSP = 2         /* Phase II by per-source SSSP on G^r (the paper's own Phase II, P:101;
+                               SURVEY 8.f NEXT 2) instead of blocked FW; same D bit for bit */
 };
 
 typedef struct ear_plan_s *ear_plan_t; /* Reduce(G) result: descriptors + reduced edge list (device) */
@@ -108,6 +110,8 @@ void ear_plan_destroy(ear_plan_t plan);
  * tiles; D is initialised here (EAR_INF, 0 diagonal, min over parallel G^r edges).
  * Layout: row-major int32, leading dimension ldd (elements, ldd >= Np and ldd % 4 == 0, d_D 16-byte
  * aligned), Np = info.n_reduced_padded; padded vertices are isolated.
+ * With EAR_FLAG_SSSP in the plan's flags, D is computed row by row by per-source label-correcting
+ * SSSP on G^r instead (sharded: every rank its own rows, no communication until the gather).
  *   comm == NULL: d_D is the full Np x Np matrix.
  *   comm != NULL: d_D is this rank's row block, rows [rank*Np/P, (rank+1)*Np/P) x all Np columns
  *                 (Np from ear_plan_info with nranks = P); the pivot row block is broadcast over
@@ -195,6 +199,9 @@ typedef struct {
   double expand_ms, same_chain_ms;
   int64_t expand_launches;
   double expand_bytes;         /* algorithmic HBM bytes of k_expand: 4*rows*n + 4*Nr^2 + 16*n */
+  double sssp_ms;              /* Phase II by per-source SSSP (EAR_FLAG_SSSP) */
+  int64_t sssp_launches;
+  double sssp_arcs;            /* sources x reduced arcs (one relaxation pass) */
 } ear_profile_t;
 
 void ear_profile_enable(int32_t on);

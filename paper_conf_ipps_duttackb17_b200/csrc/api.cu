@@ -159,6 +159,10 @@ ear_status_t apsp_reduced(ear_plan_t p, int32_t *d_D, int64_t ldd, ear_comm_t co
     return EAR_EINVAL;
   }
   cudaStream_t st = (cudaStream_t)stream;
+  if (p->flags & EAR_FLAG_SSSP) {   // rows by per-source SSSP: no inter-rank exchange in Phase II
+    const int32_t rows = Np / P, row0 = (comm ? comm->rank : 0) * rows;
+    return sssp_rows(p, d_D, ldd, Np, row0, rows, st);
+  }
   if (P == 1) {
     EAR_TRY(fw_init_D(p, d_D, ldd, Np, 0, Np, st));
     return fw_single(d_D, ldd, Np, st);

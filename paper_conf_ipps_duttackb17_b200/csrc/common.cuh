@@ -65,6 +65,11 @@ struct ear_plan_s {
   int32_t n_chain_vertices = 0;
   // reduced arcs (both directions, before the P:90 min)
   int32_t *re_u = nullptr, *re_v = nullptr, *re_w = nullptr;
+  // reduced-graph CSR for the per-source SSSP Phase II (built on first use)
+  int32_t *r_rowptr = nullptr, *r_col = nullptr, *r_w = nullptr;
+  void *r_arcs = nullptr;       // packed (col, w) int2 arcs: ELL rows of r_ell_k per vertex, or CSR order
+  int32_t r_ell_k = -1;
+  int32_t n_rarcs = 0;
 };
 
 struct ear_comm_s {
@@ -77,7 +82,7 @@ struct ear_comm_s {
 
 namespace ear {
 // prof.cu
-enum ProfKind { PK_DECOMPOSE, PK_FW_INIT, PK_FW_P1, PK_FW_P2, PK_FW_P3, PK_COMM, PK_EXPAND, PK_SAME_CHAIN };
+enum ProfKind { PK_DECOMPOSE, PK_FW_INIT, PK_FW_P1, PK_FW_P2, PK_FW_P3, PK_COMM, PK_EXPAND, PK_SAME_CHAIN, PK_SSSP };
 void count_launch(int n = 1);
 int prof_begin(int kind, cudaStream_t s);                // -1 when profiling is off
 void prof_end(int slot, cudaStream_t s, double work);
@@ -93,6 +98,9 @@ ear_status_t fw_init_D(const ear_plan_s *plan, int32_t *D, int64_t ldd, int32_t 
 ear_status_t fw_single(int32_t *D, int64_t ldd, int32_t Np, cudaStream_t stream);
 ear_status_t fw_sharded(int32_t *Dblk, int64_t ldd, int32_t Np, ear_comm_s *comm, cudaStream_t stream);
 ear_status_t fw_sharded_emulated(int32_t *D, int64_t ldd, int32_t Np, int32_t P, cudaStream_t stream);
+// sssp.cu
+ear_status_t sssp_rows(ear_plan_s *plan, int32_t *D, int64_t ldd, int32_t Np, int32_t row0, int32_t rows,
+                       cudaStream_t stream);
 // expand.cu
 ear_status_t expand(const ear_plan_s *plan, const int32_t *D, int64_t ldd, int32_t row_begin,
                     int32_t row_end, int32_t *out, int64_t ldo, cudaStream_t stream);

@@ -299,7 +299,8 @@ struct Scratch {
 // and are released in stream order on the stream the plan was created on.
 void plan_free(ear_plan_s *p) {
   if (!p) return;
-  void *arrs[] = {p->desc, p->tid, p->ear, p->seg_of, p->seg_start, p->seg_vert, p->re_u, p->re_v, p->re_w};
+  void *arrs[] = {p->desc, p->tid, p->ear, p->seg_of, p->seg_start, p->seg_vert, p->re_u, p->re_v, p->re_w,
+                  p->r_rowptr, p->r_col, p->r_w, p->r_arcs};
   for (void *a : arrs)
     if (a) cudaFreeAsync(a, p->stream);
 }

@@ -1,0 +1,452 @@
+// Phase II alternative: S^r by a single-source shortest-path computation from
+// every reduced vertex -- the paper's own Phase II formulation (Alg. 1 lines 4-7: "for each s in
+// V(G^r) do DIJKSTRA(G^r, s)") -- instead of the O(N_r^3) blocked FW.  For the sparse
+// reduced graphs of the paper's workloads, N_r * M_r * (rounds) << N_r^3.
+//
+// GPU form: one CTA per source at a time (persistent over sources).  The source's distance row is
+// the row of D itself (global, L2-resident while in use); the CTA runs a synchronous label-correcting
+// Bellman-Ford over a frontier bitmap in shared memory: every frontier vertex relaxes its arcs with
+// atomicMin on the row, improved vertices form the next frontier, until a round improves nothing.
+// The fixed point is the exact shortest-path row (integer weights >= 1), identical to the FW result.
+#include <cub/cub.cuh>
+
+#include <algorithm>
+#include <cstdio>
+#include <cstdlib>
+
+#include "common.cuh"
+
+namespace ear {
+namespace {
+
+constexpr int NT = 256;
+
+__global__ void k_r_make_keys(const int32_t *u, const int32_t *v, const int32_t *w, int64_t E, uint64_t *keys,
+                              int32_t *vals) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < E; i += (int64_t)gridDim.x * blockDim.x) {
+    keys[i] = ((uint64_t)(uint32_t)u[i] << 32) | (uint32_t)v[i];
+    vals[i] = w[i];
+  }
+}
+
+struct MinOp {
+  __device__ __forceinline__ int32_t operator()(int32_t a, int32_t b) const { return a < b ? a : b; }
+};
+
+__global__ void k_r_split(const uint64_t *keys, int64_t A, int32_t *col, int32_t *deg) {
+  for (int64_t a = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; a < A; a += (int64_t)gridDim.x * blockDim.x) {
+    col[a] = (int32_t)(keys[a] & 0xFFFFFFFFu);
+    atomicAdd(&deg[keys[a] >> 32], 1);
+  }
+}
+
+__device__ __forceinline__ int32_t ld_cg(const int32_t *p) { return __ldcg(p); }
+
+// rows [src0, src1) of D (global rows; this launch writes D + (src - row0) * ldd)
+__global__ void __launch_bounds__(NT) k_sssp_bf(const int32_t *__restrict__ rowptr, const int32_t *__restrict__ col,
+                                               const int32_t *__restrict__ wt, int32_t nr, int32_t Np, int32_t *D,
+                                               int64_t ldd, int32_t row0, int32_t src0, int32_t src1,
+                                               unsigned long long *stats) {
+  extern __shared__ uint32_t bits[];        // [2][W] frontier bitmaps
+  __shared__ int flag[3];
+  const int W = (Np + 31) >> 5;
+  const int tid = threadIdx.x;
+  unsigned long long my_rounds = 0, my_relax = 0, my_improve = 0, my_visits = 0;
+  for (int32_t src = src0 + blockIdx.x; src < src1; src += gridDim.x) {
+    int32_t *dist = D + (int64_t)(src - row0) * ldd;
+    for (int i = tid * 4; i < Np; i += NT * 4)   // Np % 4 == 0, ldd % 4 == 0
+      *reinterpret_cast<int4 *>(dist + i) = make_int4(INF, INF, INF, INF);
+    for (int w = tid; w < 2 * W; w += NT) bits[w] = 0u;
+    if (tid < 3) flag[tid] = 0;
+    __syncthreads();
+    if (tid == 0) {
+      dist[src] = 0;
+      bits[src >> 5] = 1u << (src & 31);
+    }
+    __syncthreads();
+    if (src >= nr) continue;   // padding vertex: isolated (INF row, 0 diagonal)
+    for (int it = 0;; ++it) {
+      uint32_t *cur = bits + (it & 1) * W, *nxt = bits + ((it + 1) & 1) * W;
+      if (tid == 0) flag[(it + 1) % 3] = 0;
+      for (int w = tid; w < W; w += NT) {
+        uint32_t m = cur[w];
+        if (!m) continue;
+        cur[w] = 0u;   // consumed (this word is owned by this thread in this round)
+        while (m) {
+          const int b = __ffs(m) - 1;
+          m &= m - 1;
+          const int v = (w << 5) + b;
+          ++my_visits;
+          const int32_t dv = ld_cg(dist + v);
+          const int a1 = __ldg(rowptr + v + 1);
+          for (int a = __ldg(rowptr + v); a < a1; ++a) {
+            const int u = __ldg(col + a);
+            const int32_t nd = dv + __ldg(wt + a);
+            ++my_relax;
+            if (nd < ld_cg(dist + u)) {
+              const int32_t old = atomicMin(dist + u, nd);
+              if (nd < old) {
+                ++my_improve;
+                atomicOr(&nxt[u >> 5], 1u << (u & 31));
+                flag[it % 3] = 1;
+              }
+            }
+          }
+        }
+      }
+      __syncthreads();
+      const int more = flag[it % 3];
+      ++my_rounds;
+      if (!more) break;
+    }
+    __syncthreads();
+  }
+  if (stats) {
+    if (tid == 0) atomicAdd(&stats[0], my_rounds);
+    atomicAdd(&stats[1], my_relax);
+    atomicAdd(&stats[2], my_improve);
+    atomicAdd(&stats[3], my_visits);
+  }
+}
+
+// The same label-correcting rounds with the distance row in SHARED memory (Np ints + two bitmaps +
+// a frontier list): every read-modify-write of the frontier expansion stays on-chip; the finished row
+// is streamed to D with 128-bit stores.  Each round the frontier bitmap is compacted into a list
+// (block scan of per-thread popcounts) so that every thread expands about one frontier vertex --
+// one dependent (rowptr -> arcs) global-latency chain per round instead of several.  Arcs are packed
+// (target, weight) int2 so one load fetches both.
+constexpr int SSSP_LIST = 4096;   // frontier list capacity per pass
+
+template <int NTS, int K>
+__global__ void __launch_bounds__(NTS) k_sssp_smem(const int32_t *__restrict__ rowptr, const int2 *__restrict__ arcs,
+                                                   int32_t nr, int32_t Np, int32_t *D, int64_t ldd, int32_t row0,
+                                                   int32_t src0, int32_t src1, unsigned long long *stats) {
+  extern __shared__ __align__(16) int32_t sm[];
+  int32_t *dist = sm;                                                 // [Np]
+  int32_t *list = sm + Np;                                            // [SSSP_LIST]
+  uint32_t *bits = reinterpret_cast<uint32_t *>(sm + Np + SSSP_LIST); // [2][W]
+  __shared__ int flag[3];
+  __shared__ int wsum[NTS / 32];
+  const int W = (Np + 31) >> 5;
+  const int KW = (W + NTS - 1) / NTS;       // bitmap words per thread (contiguous)
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  unsigned long long my_rounds = 0, my_relax = 0;
+  for (int32_t src = src0 + blockIdx.x; src < src1; src += gridDim.x) {
+    for (int i = tid; i < Np; i += NTS) dist[i] = INF;
+    for (int w = tid; w < 2 * W; w += NTS) bits[w] = 0u;
+    if (tid < 3) flag[tid] = 0;
+    __syncthreads();
+    if (tid == 0) {
+      dist[src] = 0;
+      bits[src >> 5] = 1u << (src & 31);
+    }
+    __syncthreads();
+    if (src < nr) {
+      for (int it = 0;; ++it) {
+        uint32_t *cur = bits + (it & 1) * W, *nxt = bits + ((it + 1) & 1) * W;
+        if (tid == 0) flag[(it + 1) % 3] = 0;
+        // 1. rank the frontier: per-thread popcount over its words, block exclusive scan
+        const int w0 = tid * KW, w1 = min(W, w0 + KW);
+        int cnt = 0;
+        for (int w = w0; w < w1; ++w) cnt += __popc(cur[w]);
+        int x = cnt;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+          const int y = __shfl_up_sync(0xffffffffu, x, o);
+          if (lane >= o) x += y;
+        }
+        if (lane == 31) wsum[warp] = x;
+        __syncthreads();
+        if (warp == 0) {
+          int v = lane < NTS / 32 ? wsum[lane] : 0;
+#pragma unroll
+          for (int o = 1; o < 32; o <<= 1) {
+            const int y = __shfl_up_sync(0xffffffffu, v, o);
+            if (lane >= o) v += y;
+          }
+          if (lane < NTS / 32) wsum[lane] = v;
+        }
+        __syncthreads();
+        const int excl = x - cnt + (warp ? wsum[warp - 1] : 0);
+        const int F = wsum[NTS / 32 - 1];
+        // 2. expand the frontier pass by pass (list capacity SSSP_LIST)
+        for (int base = 0; base < F; base += SSSP_LIST) {
+          if (excl < base + SSSP_LIST && excl + cnt > base) {
+            int r = excl;
+            for (int w = w0; w < w1; ++w) {
+              uint32_t m = cur[w];
+              while (m) {
+                const int b = __ffs(m) - 1;
+                m &= m - 1;
+                if (r >= base && r < base + SSSP_LIST) list[r - base] = (w << 5) + b;
+                ++r;
+              }
+            }
+          }
+          __syncthreads();
+          const int nb = min(SSSP_LIST, F - base);
+          if constexpr (K > 0) {
+            // ELL adjacency: vertex v's arcs are the K int2 at arcs[v*K ...] (weight INF padding), so
+            // all of a thread's vertices' arcs are fetched with independent 128-bit loads at once
+            constexpr int J = 4;   // vertices per thread per batch
+            for (int i0 = 0; i0 < nb; i0 += J * NTS) {
+              int vv[J];
+              int4 e[J][K > 0 ? K / 2 : 1];
+#pragma unroll
+              for (int j = 0; j < J; ++j) {
+                const int i = i0 + j * NTS + tid;
+                vv[j] = i < nb ? list[i] : -1;
+                const int4 *row = reinterpret_cast<const int4 *>(arcs + (int64_t)max(vv[j], 0) * K);
+#pragma unroll
+                for (int k = 0; k < K / 2; ++k)
+                  e[j][k] = vv[j] >= 0 ? __ldg(row + k) : make_int4(0, INF, 0, INF);
+              }
+#pragma unroll
+              for (int j = 0; j < J; ++j) {
+                if (vv[j] < 0) continue;
+                const int32_t dv = dist[vv[j]];
+#pragma unroll
+                for (int k = 0; k < K; ++k) {
+                  const int u = (k & 1) ? e[j][k / 2].z : e[j][k / 2].x;
+                  const int32_t nd = dv + ((k & 1) ? e[j][k / 2].w : e[j][k / 2].y);
+                  if (nd < dist[u]) {
+                    if (stats) ++my_relax;
+                    const int32_t old = atomicMin(dist + u, nd);
+                    if (nd < old) {
+                      atomicOr(&nxt[u >> 5], 1u << (u & 31));
+                      flag[it % 3] = 1;
+                    }
+                  }
+                }
+              }
+            }
+          } else {
+            for (int i = tid; i < nb; i += NTS) {
+              const int v = list[i];
+              const int32_t dv = dist[v];
+              const int a0 = __ldg(rowptr + v), a1 = __ldg(rowptr + v + 1);
+              for (int a = a0; a < a1; a += 4) {   // up to 4 independent arc loads in flight
+                int2 e[4];
+  #pragma unroll
+                for (int k = 0; k < 4; ++k) e[k] = (a + k < a1) ? __ldg(arcs + a + k) : make_int2(0, INF);
+  #pragma unroll
+                for (int k = 0; k < 4; ++k) {
+                  if (a + k < a1) {
+                    const int u = e[k].x;
+                    const int32_t nd = dv + e[k].y;
+                    if (stats) ++my_relax;
+                    if (nd < dist[u]) {
+                      const int32_t old = atomicMin(dist + u, nd);
+                      if (nd < old) {
+                        atomicOr(&nxt[u >> 5], 1u << (u & 31));
+                        flag[it % 3] = 1;
+                      }
+                    }
+                  }
+                }
+              }
+            }
+          }
+          __syncthreads();
+        }
+        // 3. the expanded frontier is consumed
+        for (int w = w0; w < w1; ++w) cur[w] = 0u;
+        const int more = flag[it % 3];
+        ++my_rounds;
+        if (!more) break;
+      }
+    }
+    __syncthreads();
+    int32_t *row = D + (int64_t)(src - row0) * ldd;
+    for (int i = tid * 4; i < Np; i += NTS * 4)   // Np % 4 == 0, 16-byte aligned rows
+      *reinterpret_cast<int4 *>(row + i) = *reinterpret_cast<const int4 *>(dist + i);
+    __syncthreads();
+  }
+  if (stats) {
+    if (tid == 0) atomicAdd(&stats[0], my_rounds);
+    atomicAdd(&stats[1], my_relax);
+  }
+}
+
+__global__ void k_build_ell(const int32_t *rowptr, const int32_t *col, const int32_t *w, int32_t nr, int K,
+                            int2 *ell) {
+  for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < nr; v += (int64_t)gridDim.x * blockDim.x) {
+    const int a0 = rowptr[v], d = rowptr[v + 1] - a0;
+    for (int k = 0; k < K; ++k) ell[v * K + k] = k < d ? make_int2(col[a0 + k], w[a0 + k]) : make_int2(0, INF);
+  }
+}
+
+__global__ void k_max_deg(const int32_t *rowptr, int32_t nr, int32_t *out) {
+  int m = 0;
+  for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < nr; v += (int64_t)gridDim.x * blockDim.x)
+    m = max(m, rowptr[v + 1] - rowptr[v]);
+  atomicMax(out, m);
+}
+
+__global__ void k_pack_arcs(const int32_t *col, const int32_t *w, int32_t A, int2 *arcs) {
+  for (int64_t a = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; a < A; a += (int64_t)gridDim.x * blockDim.x)
+    arcs[a] = make_int2(col[a], w[a]);
+}
+
+}  // namespace
+
+// Reduced-graph CSR (parallel G^r arcs -> minimum weight), built once per plan.
+ear_status_t sssp_prepare(ear_plan_s *p, cudaStream_t st) {
+  if (p->r_rowptr) return EAR_OK;
+  const int64_t E = p->n_redges;
+  const int32_t nr = p->n_reduced;
+  uint64_t *k0 = nullptr, *k1 = nullptr, *uk = nullptr;
+  int32_t *v0 = nullptr, *v1 = nullptr, *uv = nullptr, *nruns = nullptr, *deg = nullptr;
+  void *tmp = nullptr;
+  size_t tb1 = 0, tb2 = 0, tb3 = 0;
+  const int64_t E1 = std::max<int64_t>(E, 1);
+  auto alloc = [&](void **q, size_t b) { return cudaMallocAsync(q, std::max<size_t>(b, 16), st); };
+  cudaError_t e = cudaSuccess;
+  e = alloc((void **)&k0, 8 * E1); if (e == cudaSuccess) e = alloc((void **)&k1, 8 * E1);
+  if (e == cudaSuccess) e = alloc((void **)&uk, 8 * E1);
+  if (e == cudaSuccess) e = alloc((void **)&v0, 4 * E1);
+  if (e == cudaSuccess) e = alloc((void **)&v1, 4 * E1);
+  if (e == cudaSuccess) e = alloc((void **)&uv, 4 * E1);
+  if (e == cudaSuccess) e = alloc((void **)&nruns, 4);
+  if (e == cudaSuccess) e = alloc((void **)&deg, 4 * ((size_t)nr + 1));
+  if (e != cudaSuccess) { set_error("sssp_prepare: %s", cudaGetErrorString(e)); return EAR_ENOMEM; }
+  int32_t A = 0;
+  if (E > 0) {
+    const int g = (int)std::min<int64_t>(ceil_div(E, 256), 4096);
+    EAR_LAUNCH(k_r_make_keys, g, 256, 0, st)(p->re_u, p->re_v, p->re_w, E, k0, v0);
+    cub::DoubleBuffer<uint64_t> dk(k0, k1);
+    cub::DoubleBuffer<int32_t> dv(v0, v1);
+    int bits = 1;
+    while ((1ll << bits) < nr) ++bits;
+    cub::DeviceRadixSort::SortPairs(nullptr, tb1, dk, dv, (int)E, 0, 32 + bits, st);
+    cub::DeviceReduce::ReduceByKey(nullptr, tb2, k0, uk, v0, uv, nruns, MinOp(), (int)E, st);
+    cub::DeviceScan::ExclusiveSum(nullptr, tb3, deg, deg, nr + 1, st);
+    EAR_CUDA_TRY(cudaMallocAsync(&tmp, std::max({tb1, tb2, tb3, (size_t)16}), st));
+    EAR_CUDA_TRY(cub::DeviceRadixSort::SortPairs(tmp, tb1, dk, dv, (int)E, 0, 32 + bits, st));
+    EAR_CUDA_TRY(cub::DeviceReduce::ReduceByKey(tmp, tb2, dk.Current(), uk, dv.Current(), uv, nruns, MinOp(), (int)E,
+                                                st));
+    EAR_CUDA_TRY(cudaMemcpyAsync(&A, nruns, 4, cudaMemcpyDeviceToHost, st));
+    EAR_CUDA_TRY(cudaStreamSynchronize(st));
+  }
+  EAR_CUDA_TRY(cudaMallocAsync((void **)&p->r_rowptr, 4 * ((size_t)nr + 1), st));
+  EAR_CUDA_TRY(cudaMallocAsync((void **)&p->r_col, 4 * (size_t)std::max(A, 1), st));
+  EAR_CUDA_TRY(cudaMallocAsync((void **)&p->r_w, 4 * (size_t)std::max(A, 1), st));
+  EAR_CUDA_TRY(cudaMemsetAsync(deg, 0, 4 * ((size_t)nr + 1), st));
+  if (A > 0) {
+    const int g = (int)std::min<int64_t>(ceil_div(A, 256), 4096);
+    EAR_LAUNCH(k_r_split, g, 256, 0, st)(uk, A, p->r_col, deg);
+    EAR_CUDA_TRY(cudaMemcpyAsync(p->r_w, uv, 4 * (size_t)A, cudaMemcpyDeviceToDevice, st));
+    EAR_CUDA_TRY(cub::DeviceScan::ExclusiveSum(tmp, tb3, deg, p->r_rowptr, nr + 1, st));
+  } else {
+    EAR_CUDA_TRY(cudaMemsetAsync(p->r_rowptr, 0, 4 * ((size_t)nr + 1), st));
+  }
+  p->n_rarcs = A;
+  void *fr[] = {k0, k1, uk, v0, v1, uv, nruns, deg, tmp};
+  for (void *q : fr)
+    if (q) cudaFreeAsync(q, st);
+  EAR_CUDA_TRY(cudaGetLastError());
+  return EAR_OK;
+}
+
+template <int NTS, int K>
+static ear_status_t sssp_launch(ear_plan_s *p, int32_t *D, int64_t ldd, int32_t Np, int32_t row0, int32_t rows,
+                                int smem_s, int nsm, unsigned long long *d_stats, cudaStream_t st) {
+  static int attr_s = 0;
+  if (smem_s > attr_s) {
+    EAR_CUDA_TRY(cudaFuncSetAttribute(k_sssp_smem<NTS, K>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_s));
+    attr_s = smem_s;
+  }
+  int per_sm = 1;
+  EAR_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_sssp_smem<NTS, K>, NTS, smem_s));
+  const int64_t grid = std::min<int64_t>(rows, (int64_t)nsm * std::max(per_sm, 1));
+  int s = prof_begin(PK_SSSP, st);
+  EAR_LAUNCH((k_sssp_smem<NTS, K>), (unsigned)grid, NTS, smem_s, st)(
+      p->r_rowptr, reinterpret_cast<const int2 *>(p->r_arcs), p->n_reduced, Np, D, ldd, row0, row0, row0 + rows,
+      d_stats);
+  prof_end(s, st, (double)rows * (double)p->n_rarcs);
+  if (d_stats) {
+    unsigned long long h[4];
+    EAR_CUDA_TRY(cudaMemcpyAsync(h, d_stats, 32, cudaMemcpyDeviceToHost, st));
+    EAR_CUDA_TRY(cudaStreamSynchronize(st));
+    fprintf(stderr, "[sssp smem K=%d] grid=%lld per_sm=%d rows=%d rounds=%.1f/source relax=%.0f/source arcs=%d\n", K,
+            (long long)grid, per_sm, rows, (double)h[0] / rows, (double)h[1] / rows, p->n_rarcs);
+  }
+  EAR_CUDA_TRY(cudaGetLastError());
+  return EAR_OK;
+}
+
+// Rows [row0, row0 + rows) of D (row-major, ldd) by per-source Bellman-Ford on G^r.
+ear_status_t sssp_rows(ear_plan_s *p, int32_t *D, int64_t ldd, int32_t Np, int32_t row0, int32_t rows,
+                       cudaStream_t st) {
+  EAR_TRY(sssp_prepare(p, st));
+  if (rows <= 0) return EAR_OK;
+  const int W = (Np + 31) / 32;
+  static unsigned long long *d_stats = nullptr;
+  static const bool want_stats = getenv("EAR_SSSP_STATS") != nullptr;
+  if (want_stats && !d_stats) EAR_CUDA_TRY(cudaMalloc((void **)&d_stats, 32));
+  if (want_stats) EAR_CUDA_TRY(cudaMemsetAsync(d_stats, 0, 32, st));
+  int dev = 0, nsm = 148;
+  EAR_CUDA_TRY(cudaGetDevice(&dev));
+  EAR_CUDA_TRY(cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev));
+  int max_smem = 0;
+  EAR_CUDA_TRY(cudaDeviceGetAttribute(&max_smem, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev));
+  const int smem_s = 4 * Np + 4 * SSSP_LIST + 8 * W;
+  if (smem_s + 64 <= max_smem && !getenv("EAR_SSSP_GLOBAL")) {
+    // distance row on chip; adjacency as ELL rows of K arcs when the max degree allows (else CSR)
+    if (!p->r_arcs) {
+      int32_t *d_md = nullptr, md = 0;
+      EAR_CUDA_TRY(cudaMallocAsync((void **)&d_md, 4, st));
+      EAR_CUDA_TRY(cudaMemsetAsync(d_md, 0, 4, st));
+      EAR_LAUNCH(k_max_deg, (int)std::min<int64_t>(ceil_div(p->n_reduced, 256), 4096), 256, 0, st)(
+          p->r_rowptr, p->n_reduced, d_md);
+      EAR_CUDA_TRY(cudaMemcpyAsync(&md, d_md, 4, cudaMemcpyDeviceToHost, st));
+      EAR_CUDA_TRY(cudaStreamSynchronize(st));
+      cudaFreeAsync(d_md, st);
+      p->r_ell_k = md <= 4 ? 4 : md <= 8 ? 8 : md <= 12 ? 12 : md <= 16 ? 16 : 0;
+      if (p->r_ell_k > 0) {
+        EAR_CUDA_TRY(cudaMallocAsync((void **)&p->r_arcs, sizeof(int2) * (size_t)p->r_ell_k * std::max(p->n_reduced, 1), st));
+        EAR_LAUNCH(k_build_ell, (int)std::min<int64_t>(ceil_div(p->n_reduced, 256), 4096), 256, 0, st)(
+            p->r_rowptr, p->r_col, p->r_w, p->n_reduced, p->r_ell_k, reinterpret_cast<int2 *>(p->r_arcs));
+      } else {
+        EAR_CUDA_TRY(cudaMallocAsync((void **)&p->r_arcs, sizeof(int2) * (size_t)std::max(p->n_rarcs, 1), st));
+        if (p->n_rarcs > 0)
+          EAR_LAUNCH(k_pack_arcs, (int)std::min<int64_t>(ceil_div(p->n_rarcs, 256), 4096), 256, 0, st)(
+              p->r_col, p->r_w, p->n_rarcs, reinterpret_cast<int2 *>(p->r_arcs));
+      }
+    }
+    constexpr int NTS = 512;
+    switch (p->r_ell_k) {
+      case 4: return sssp_launch<NTS, 4>(p, D, ldd, Np, row0, rows, smem_s, nsm, want_stats ? d_stats : nullptr, st);
+      case 8: return sssp_launch<NTS, 8>(p, D, ldd, Np, row0, rows, smem_s, nsm, want_stats ? d_stats : nullptr, st);
+      case 12: return sssp_launch<NTS, 12>(p, D, ldd, Np, row0, rows, smem_s, nsm, want_stats ? d_stats : nullptr, st);
+      case 16: return sssp_launch<NTS, 16>(p, D, ldd, Np, row0, rows, smem_s, nsm, want_stats ? d_stats : nullptr, st);
+      default: return sssp_launch<NTS, 0>(p, D, ldd, Np, row0, rows, smem_s, nsm, want_stats ? d_stats : nullptr, st);
+    }
+  }
+  const int smem = 2 * W * 4;
+  static int attr = 0;
+  if (smem > attr) {
+    EAR_CUDA_TRY(cudaFuncSetAttribute(k_sssp_bf, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+    attr = smem;
+  }
+  int per_sm = 1;
+  EAR_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_sssp_bf, NT, smem));
+  // concurrent rows live in L2: cap the number of resident sources (rows of 4*Np bytes) near 96 MB
+  const int64_t l2_rows = std::max<int64_t>(nsm, (96ll << 20) / (4ll * Np));
+  const int64_t grid = std::min<int64_t>({(int64_t)rows, (int64_t)nsm * std::max(per_sm, 1), l2_rows});
+  int s = prof_begin(PK_SSSP, st);
+  EAR_LAUNCH(k_sssp_bf, (unsigned)grid, NT, smem, st)(p->r_rowptr, p->r_col, p->r_w, p->n_reduced, Np, D, ldd, row0,
+                                                      row0, row0 + rows, want_stats ? d_stats : nullptr);
+  if (want_stats) {
+    unsigned long long h[4];
+    EAR_CUDA_TRY(cudaMemcpyAsync(h, d_stats, 32, cudaMemcpyDeviceToHost, st));
+    EAR_CUDA_TRY(cudaStreamSynchronize(st));
+    fprintf(stderr, "[sssp] grid=%lld rows=%d rounds=%llu (%.1f/source) relax=%llu (%.0f/source) improve=%llu visits=%llu arcs=%d\n",
+            (long long)grid, rows, h[0], (double)h[0] / rows, h[1], (double)h[1] / rows, h[2], h[3], p->n_rarcs);
+  }
+  prof_end(s, st, (double)rows * (double)p->n_rarcs);
+  EAR_CUDA_TRY(cudaGetLastError());
+  return EAR_OK;
+}
+
+}  // namespace ear

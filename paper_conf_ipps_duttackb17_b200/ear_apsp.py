@@ -26,6 +26,7 @@ INF = 0x3FFFFFFF
 TILE = 128
 FLAG_NONE = 0
 FLAG_NO_CONTRACT = 1
+FLAG_SSSP = 2
 
 _lib = None
 
@@ -48,7 +49,8 @@ class _Profile(ctypes.Structure):
                 ("fw_phase3_launches", ctypes.c_int64), ("fw_phase2_minplus", ctypes.c_double),
                 ("fw_phase3_minplus", ctypes.c_double), ("comm_ms", ctypes.c_double), ("expand_ms", ctypes.c_double),
                 ("same_chain_ms", ctypes.c_double), ("expand_launches", ctypes.c_int64),
-                ("expand_bytes", ctypes.c_double)]
+                ("expand_bytes", ctypes.c_double), ("sssp_ms", ctypes.c_double), ("sssp_launches", ctypes.c_int64),
+                ("sssp_arcs", ctypes.c_double)]
 
 
 # (name, restype, argtypes) for every symbol declared in include/ear_apsp.h

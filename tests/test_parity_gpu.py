@@ -302,3 +302,40 @@ def test_query_pairs_cfg4_without_full_matrix(pkg):
     t = np.tile(cols, len(rows)).astype(np.int32)
     got = pkg.query_pairs(plan, D, dev(s), dev(t)).cpu().numpy().reshape(len(rows), len(cols))
     assert_exact(got, ref[:, cols], "cfg4 query pairs")
+
+
+# ------------------------------------------------------------------------------ NEXT 2: SSSP Phase II
+@pytest.mark.parametrize("seed", range(12))
+def test_sssp_phase2_corner_cases(pkg, seed):
+    g = gg.corner_cases(3000 + seed, n_target=30 + 40 * seed)
+    assert_exact(run_full(pkg, g, flags=pkg.FLAG_SSSP), oracle.apsp(g.n, g.src, g.dst, g.w), f"sssp seed {seed}")
+
+
+@pytest.mark.parametrize("name", ["cfg1", "cfg2"])
+def test_sssp_D_equals_fw_D(pkg, name):
+    """Per-source SSSP on G^r (the paper's Phase II) and blocked FW give the same D bit for bit."""
+    g = gg.config(name)
+    p1 = pkg.ear_decompose(g.n, dev(g.src), dev(g.dst), dev(g.w))
+    p2 = pkg.ear_decompose(g.n, dev(g.src), dev(g.dst), dev(g.w), flags=pkg.FLAG_SSSP)
+    D1 = pkg.alloc_D(p1)
+    D2 = pkg.alloc_D(p2)
+    pkg.apsp_reduced(p1, D1)
+    pkg.apsp_reduced(p2, D2)
+    torch.cuda.synchronize()
+    assert torch.equal(D1, D2)
+
+
+def test_sssp_cfg4_sampled_rows(pkg):
+    g = gg.config("cfg4")
+    out = pkg.apsp_full(g.n, dev(g.src), dev(g.dst), dev(g.w), flags=pkg.FLAG_SSSP)
+    rows = np.unique(np.concatenate([[0, g.n - 1], np.random.default_rng(8).choice(g.n, 30, replace=False)]))
+    ref = oracle.apsp_rows(g.n, g.src, g.dst, g.w, rows)
+    assert_exact(out[torch.as_tensor(rows).cuda().long()].cpu().numpy(), ref, "cfg4 sssp rows")
+    del out
+    torch.cuda.empty_cache()
+
+
+@pytest.mark.parametrize("case", ["n1", "m0", "cycle", "path"])
+def test_sssp_degenerate(pkg, case):
+    g = {"n1": graph(1, []), "m0": graph(7, []), "cycle": gg.cycle(9, seed=5), "path": gg.path(40, seed=6)}[case]
+    assert_exact(run_full(pkg, g, flags=pkg.FLAG_SSSP), oracle.apsp(g.n, g.src, g.dst, g.w), case)
