@@ -268,6 +268,119 @@ __global__ void __launch_bounds__(NTS) k_sssp_smem(const int32_t *__restrict__ r
   }
 }
 
+// List-driven rounds with ONE barrier per round (ELL adjacency, K arcs per vertex row).  Round r
+// expands list L[r%2] and appends improved vertices to L[(r+1)%2]; membership bitmaps M[.] dedupe the
+// appends (set on append, cleared by whoever expands the vertex), and the list counters rotate over
+// three slots so that every reset happens in a round where nobody reads or appends that slot.  If a
+// round's appends exceed the list capacity, the next round falls back to scanning its bitmap.
+template <int NTS, int K>
+__global__ void __launch_bounds__(NTS) k_sssp_list(const int2 *__restrict__ ell, int32_t nr, int32_t Np, int32_t *D,
+                                                   int64_t ldd, int32_t row0, int32_t src0, int32_t src1, int cap,
+                                                   unsigned long long *stats) {
+  extern __shared__ __align__(16) int32_t sm[];
+  const int W = (Np + 31) >> 5;
+  int32_t *dist = sm;                                               // [Np]
+  int32_t *L0 = sm + Np;                                            // [cap]
+  int32_t *L1 = L0 + cap;                                           // [cap]
+  uint32_t *M0 = reinterpret_cast<uint32_t *>(L1 + cap);            // [W]
+  uint32_t *M1 = M0 + W;                                            // [W]
+  __shared__ int cnt[3], ovf[3];
+  const int tid = threadIdx.x;
+  unsigned long long my_rounds = 0, my_relax = 0;
+  for (int32_t src = src0 + blockIdx.x; src < src1; src += gridDim.x) {
+    for (int i = tid; i < Np; i += NTS) dist[i] = INF;
+    for (int w = tid; w < 2 * W; w += NTS) M0[w] = 0u;
+    if (tid < 3) { cnt[tid] = 0; ovf[tid] = 0; }
+    __syncthreads();
+    if (tid == 0) {
+      dist[src] = 0;
+      L0[0] = src;
+      M0[src >> 5] = 1u << (src & 31);
+      cnt[0] = 1;
+    }
+    __syncthreads();
+    if (src < nr) {
+      for (int r = 0;; ++r) {
+        int32_t *Lc = (r & 1) ? L1 : L0, *Ln = (r & 1) ? L0 : L1;
+        uint32_t *Mc = (r & 1) ? M1 : M0, *Mn = (r & 1) ? M0 : M1;
+        const int n = cnt[r % 3];
+        const bool scan = ovf[r % 3] != 0;
+        int *ncnt = &cnt[(r + 1) % 3];
+        int *novf = &ovf[(r + 1) % 3];
+        if (tid == 0) { cnt[(r + 2) % 3] = 0; ovf[(r + 2) % 3] = 0; }
+        auto relax_from = [&](int v, const int4 *e) {
+          const int32_t dv = dist[v];
+#pragma unroll
+          for (int k = 0; k < K; ++k) {
+            const int u = (k & 1) ? e[k / 2].z : e[k / 2].x;
+            const int32_t nd = dv + ((k & 1) ? e[k / 2].w : e[k / 2].y);
+            if (nd < dist[u]) {
+              if (stats) ++my_relax;
+              const int32_t old = atomicMin(dist + u, nd);
+              if (nd < old) {
+                const uint32_t bit = 1u << (u & 31);
+                if (!(atomicOr(&Mn[u >> 5], bit) & bit)) {
+                  const int idx = atomicAdd(ncnt, 1);
+                  if (idx < cap) Ln[idx] = u; else *novf = 1;
+                }
+              }
+            }
+          }
+        };
+        if (!scan) {
+          constexpr int J = 4;   // vertices per thread per batch: their arc rows load together
+          for (int i0 = 0; i0 < n; i0 += J * NTS) {
+            int vv[J];
+            int4 e[J][K / 2];
+#pragma unroll
+            for (int j = 0; j < J; ++j) {
+              const int i = i0 + j * NTS + tid;
+              vv[j] = i < n ? Lc[i] : -1;
+              const int4 *row = reinterpret_cast<const int4 *>(ell + (int64_t)max(vv[j], 0) * K);
+#pragma unroll
+              for (int k = 0; k < K / 2; ++k) e[j][k] = vv[j] >= 0 ? __ldg(row + k) : make_int4(0, INF, 0, INF);
+            }
+#pragma unroll
+            for (int j = 0; j < J; ++j) {
+              if (vv[j] < 0) continue;
+              atomicAnd(&Mc[vv[j] >> 5], ~(1u << (vv[j] & 31)));
+              relax_from(vv[j], e[j]);
+            }
+          }
+        } else {   // overflowed list: the bitmap holds the frontier
+          for (int w = tid; w < W; w += NTS) {
+            uint32_t m = Mc[w];
+            if (!m) continue;
+            atomicAnd(&Mc[w], ~m);
+            while (m) {
+              const int b = __ffs(m) - 1;
+              m &= m - 1;
+              const int v = (w << 5) + b;
+              int4 e[K / 2];
+              const int4 *row = reinterpret_cast<const int4 *>(ell + (int64_t)v * K);
+#pragma unroll
+              for (int k = 0; k < K / 2; ++k) e[k] = __ldg(row + k);
+              relax_from(v, e);
+            }
+          }
+        }
+        __syncthreads();
+        ++my_rounds;
+        if (cnt[(r + 1) % 3] == 0 && ovf[(r + 1) % 3] == 0) break;
+      }
+    }
+    __syncthreads();
+    int32_t *row = D + (int64_t)(src - row0) * ldd;
+    for (int i = tid * 4; i < Np; i += NTS * 4)   // Np % 4 == 0, 16-byte aligned rows
+      *reinterpret_cast<int4 *>(row + i) = *reinterpret_cast<const int4 *>(dist + i);
+    __syncthreads();
+  }
+  if (stats) {
+    if (tid == 0) atomicAdd(&stats[0], my_rounds);
+    atomicAdd(&stats[1], my_relax);
+  }
+}
+
 __global__ void k_build_ell(const int32_t *rowptr, const int32_t *col, const int32_t *w, int32_t nr, int K,
                             int2 *ell) {
   for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < nr; v += (int64_t)gridDim.x * blockDim.x) {
@@ -375,6 +488,36 @@ static ear_status_t sssp_launch(ear_plan_s *p, int32_t *D, int64_t ldd, int32_t 
   return EAR_OK;
 }
 
+template <int NTS, int K>
+static ear_status_t sssp_list_launch(ear_plan_s *p, int32_t *D, int64_t ldd, int32_t Np, int32_t row0, int32_t rows,
+                                     int max_smem, int nsm, unsigned long long *d_stats, cudaStream_t st) {
+  const int W = (Np + 31) / 32;
+  const int fixed = 4 * Np + 8 * W + 64;
+  const int cap = std::min(Np, (max_smem - fixed) / 8);
+  const int smem = 4 * Np + 8 * cap + 8 * W;
+  static int attr = 0;
+  if (smem > attr) {
+    EAR_CUDA_TRY(cudaFuncSetAttribute(k_sssp_list<NTS, K>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+    attr = smem;
+  }
+  int per_sm = 1;
+  EAR_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_sssp_list<NTS, K>, NTS, smem));
+  const int64_t grid = std::min<int64_t>(rows, (int64_t)nsm * std::max(per_sm, 1));
+  int s = prof_begin(PK_SSSP, st);
+  EAR_LAUNCH((k_sssp_list<NTS, K>), (unsigned)grid, NTS, smem, st)(
+      reinterpret_cast<const int2 *>(p->r_arcs), p->n_reduced, Np, D, ldd, row0, row0, row0 + rows, cap, d_stats);
+  prof_end(s, st, (double)rows * (double)p->n_rarcs);
+  if (d_stats) {
+    unsigned long long h[4];
+    EAR_CUDA_TRY(cudaMemcpyAsync(h, d_stats, 32, cudaMemcpyDeviceToHost, st));
+    EAR_CUDA_TRY(cudaStreamSynchronize(st));
+    fprintf(stderr, "[sssp list K=%d cap=%d] grid=%lld per_sm=%d rows=%d rounds=%.1f/source relax=%.0f/source\n", K,
+            cap, (long long)grid, per_sm, rows, (double)h[0] / rows, (double)h[1] / rows);
+  }
+  EAR_CUDA_TRY(cudaGetLastError());
+  return EAR_OK;
+}
+
 // Rows [row0, row0 + rows) of D (row-major, ldd) by per-source Bellman-Ford on G^r.
 ear_status_t sssp_rows(ear_plan_s *p, int32_t *D, int64_t ldd, int32_t Np, int32_t row0, int32_t rows,
                        cudaStream_t st) {
@@ -391,7 +534,7 @@ ear_status_t sssp_rows(ear_plan_s *p, int32_t *D, int64_t ldd, int32_t Np, int32
   int max_smem = 0;
   EAR_CUDA_TRY(cudaDeviceGetAttribute(&max_smem, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev));
   const int smem_s = 4 * Np + 4 * SSSP_LIST + 8 * W;
-  if (smem_s + 64 <= max_smem && !getenv("EAR_SSSP_GLOBAL")) {
+  if (smem_s + 64 <= max_smem) {
     // distance row on chip; adjacency as ELL rows of K arcs when the max degree allows (else CSR)
     if (!p->r_arcs) {
       int32_t *d_md = nullptr, md = 0;
@@ -415,6 +558,18 @@ ear_status_t sssp_rows(ear_plan_s *p, int32_t *D, int64_t ldd, int32_t Np, int32
       }
     }
     constexpr int NTS = 512;
+    // list-driven rounds win when two or more sources share an SM (cfg2: 6.7 vs 10.7 ms); with one
+    // resident source per SM the bitmap-scan rounds are faster (cfg4: 475 vs 533 ms)
+    const int list_smem = 4 * Np + 8 * std::min(Np, (max_smem - (4 * Np + 8 * W + 64)) / 8) + 8 * W;
+    if (2 * list_smem + 2048 <= max_smem + 1024) {
+      switch (p->r_ell_k) {
+        case 4: return sssp_list_launch<NTS, 4>(p, D, ldd, Np, row0, rows, max_smem, nsm, want_stats ? d_stats : nullptr, st);
+        case 8: return sssp_list_launch<NTS, 8>(p, D, ldd, Np, row0, rows, max_smem, nsm, want_stats ? d_stats : nullptr, st);
+        case 12: return sssp_list_launch<NTS, 12>(p, D, ldd, Np, row0, rows, max_smem, nsm, want_stats ? d_stats : nullptr, st);
+        case 16: return sssp_list_launch<NTS, 16>(p, D, ldd, Np, row0, rows, max_smem, nsm, want_stats ? d_stats : nullptr, st);
+        default: break;
+      }
+    }
     switch (p->r_ell_k) {
       case 4: return sssp_launch<NTS, 4>(p, D, ldd, Np, row0, rows, smem_s, nsm, want_stats ? d_stats : nullptr, st);
       case 8: return sssp_launch<NTS, 8>(p, D, ldd, Np, row0, rows, smem_s, nsm, want_stats ? d_stats : nullptr, st);
