@@ -1,0 +1,24 @@
+"""Small end-to-end runs for compute-sanitizer (memcheck / racecheck / synccheck): every kernel of the
+library on graphs small enough for the instrumented run -- FW (single + emulated sharding), SSSP,
+expansion (aligned and scalar store paths), query mode, Phase I with pure cycles."""
+import sys
+
+import numpy as np
+import torch
+
+sys.path.insert(0, ".")
+import paper_conf_ipps_duttackb17_b200 as ea  # noqa: E402
+from paper_conf_ipps_duttackb17_b200 import graphgen as gg  # noqa: E402
+
+dev = lambda a: torch.as_tensor(np.ascontiguousarray(a, dtype=np.int32)).cuda()  # noqa: E731
+for g in [gg.corner_cases(5, n_target=300), gg.torus(12, 12, 150, seed=1), gg.cycle(40, seed=2)]:
+    for flags in (0, ea.FLAG_SSSP):
+        out = ea.apsp_full(g.n, dev(g.src), dev(g.dst), dev(g.w), flags=flags)
+    plan = ea.ear_decompose(g.n, dev(g.src), dev(g.dst), dev(g.w))
+    D = ea.apsp_reduced_emulated(plan, 2)
+    big = torch.zeros((g.n, g.n + 3), dtype=torch.int32, device="cuda")
+    ea.expand_ears(plan, D, 0, g.n, out=big[:, 1:1 + g.n])
+    s = dev(np.arange(g.n)); t = dev(np.arange(g.n)[::-1].copy())
+    ea.query_pairs(plan, D, s, t)
+torch.cuda.synchronize()
+print("sanitize run ok")
