@@ -163,10 +163,11 @@ ear_status_t apsp_reduced(ear_plan_t p, int32_t *d_D, int64_t ldd, ear_comm_t co
     const int32_t rows = Np / P, row0 = (comm ? comm->rank : 0) * rows;
     return sssp_rows(p, d_D, ldd, Np, row0, rows, st);
   }
-  if (P == 1) {
+  if (!comm) {
     EAR_TRY(fw_init_D(p, d_D, ldd, Np, 0, Np, st));
     return fw_single(d_D, ldd, Np, st);
   }
+  // with a communicator -- even one of a single rank -- the row-block schedule and its NCCL calls run
   const int32_t rows = Np / P, row0 = comm->rank * rows;
   EAR_TRY(fw_init_D(p, d_D, ldd, Np, row0, rows, st));
   return fw_sharded(d_D, ldd, Np, comm, st);
@@ -194,7 +195,7 @@ ear_status_t ear_gather_reduced(ear_plan_t p, const int32_t *d_D_block, int64_t 
   const int32_t rows = Np / P;
   const int32_t rank = comm ? comm->rank : 0;
   if (ldd_block < Np || ldd_full < Np) { set_error("ear_gather_reduced: leading dimension < Np"); return EAR_EINVAL; }
-  if (P == 1) {
+  if (!comm) {
     if (d_D_block != d_D_full)
       EAR_CUDA_TRY(cudaMemcpy2DAsync(d_D_full, sizeof(int32_t) * ldd_full, d_D_block, sizeof(int32_t) * ldd_block,
                                      sizeof(int32_t) * Np, Np, cudaMemcpyDeviceToDevice, st));
@@ -248,7 +249,7 @@ static ear_status_t solve_rows(ear_plan_s *p, int32_t row_begin, int32_t row_end
   const int32_t Np = padded(p, P);
   int32_t *D = nullptr, *Dfull = nullptr;
   ear_status_t s = EAR_OK;
-  if (P == 1) {
+  if (!comm) {
     EAR_CUDA_TRY(cudaMallocAsync((void **)&D, sizeof(int32_t) * (size_t)Np * Np, st));
     s = apsp_reduced(p, D, Np, nullptr, st);
     Dfull = D;

@@ -17,7 +17,6 @@ namespace ear {
   } while (0)
 
 ear_status_t comm_bcast(ear_comm_s *comm, int32_t *buf, int64_t count, int32_t root, cudaStream_t st) {
-  if (comm->nranks == 1) return EAR_OK;
   EAR_NCCL_TRY(ncclBroadcast(buf, buf, (size_t)count, ncclInt32, root, (ncclComm_t)comm->nccl, st));
   return EAR_OK;
 }

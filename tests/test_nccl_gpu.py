@@ -1,0 +1,42 @@
+"""The NCCL path on one GPU: a communicator of ONE rank (torch.distributed nccl process group, NCCL
+unique id from the library) runs the row-block schedule with its real ncclBroadcast per FW round and
+ncclAllGather of D, then the expansion -- bit-exact against the oracle.  (The multi-rank schedule
+itself is checked on one GPU by test_parity_gpu.py::test_sharded_schedule_emulated.)"""
+import os
+import socket
+import subprocess
+import sys
+
+import pytest
+
+pytestmark = pytest.mark.gpu
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+SCRIPT = r'''
+import os, sys, numpy as np, torch, torch.distributed as dist
+sys.path.insert(0, ROOT)
+import oracle, paper_conf_ipps_duttackb17_b200 as ea
+from paper_conf_ipps_duttackb17_b200 import graphgen as gg
+torch.cuda.set_device(0)
+dist.init_process_group("nccl", rank=0, world_size=1, device_id=torch.device("cuda", 0))
+comm = ea.Comm.from_torch_distributed()
+dev = lambda a: torch.as_tensor(np.ascontiguousarray(a, dtype=np.int32)).cuda()
+for g in [gg.config("cfg1"), gg.corner_cases(12, n_target=500)]:
+    out = ea.apsp_full(g.n, dev(g.src), dev(g.dst), dev(g.w), comm=comm)
+    torch.cuda.synchronize()
+    ref = oracle.apsp(g.n, g.src, g.dst, g.w)
+    assert np.array_equal(out.cpu().numpy(), ref), "nccl path mismatch"
+    host = ea.apsp_full_host(g.n, g.src, g.dst, g.w, comm=comm)
+    assert np.array_equal(host.numpy(), ref), "nccl host path mismatch"
+comm.destroy()
+dist.destroy_process_group()
+print("NCCL-PATH-OK")
+'''
+
+
+def test_one_rank_nccl_path():
+    s = socket.socket(); s.bind(("127.0.0.1", 0)); port = s.getsockname()[1]; s.close()
+    env = dict(os.environ, MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    r = subprocess.run([sys.executable, "-c", SCRIPT.replace("ROOT", repr(ROOT))], env=env, capture_output=True,
+                       text=True, timeout=600)
+    assert "NCCL-PATH-OK" in r.stdout, r.stdout[-2000:] + r.stderr[-4000:]
