@@ -113,23 +113,34 @@ void ear_plan_destroy(ear_plan_t plan);
  * With EAR_FLAG_SSSP in the plan's flags, D is computed row by row by per-source label-correcting
  * SSSP on G^r instead (sharded: every rank its own rows, no communication until the gather).
  *   comm == NULL: d_D is the full Np x Np matrix.
- *   comm != NULL: d_D is this rank's row block, rows [rank*Np/P, (rank+1)*Np/P) x all Np columns
- *                 (Np from ear_plan_info with nranks = P); the pivot row block is broadcast over
- *                 NCCL each round.
+ *   comm != NULL (P ranks, even P = 1): d_D holds this rank's OWNED TILE ROWS -- the 128-row blocks
+ *                 ti with (ti mod 2P) in {rank, 2P-1-rank} (a zig-zag that balances the upper
+ *                 triangle), in ascending order, ear_owned_tile_rows() blocks of 128 rows x ldd.  Each
+ *                 round the pivot row block is assembled on every rank by an NCCL all-reduce(MIN) of
+ *                 the owners' pieces, closed locally, and every rank updates only its owned UPPER
+ *                 tiles: the single-GPU symmetric halving of the work survives the sharding
+ *                 (DESIGN.md "Multi-GPU").  Only the upper tiles of d_D are meaningful afterwards;
+ *                 ear_gather_reduced assembles the full symmetric matrix.
  * Asynchronous.  Errors: EAR_EINVAL (ldd too small/misaligned), EAR_ENCCL, EAR_ECUDA. */
 ear_status_t apsp_reduced(ear_plan_t plan, int32_t *d_D, int64_t ldd, ear_comm_t comm, void *stream);
 
-/* The row-block-sharded schedule of apsp_reduced for `nranks` ranks, emulated in ONE process on the
- * current device: the same per-rank kernels and addressing, rank r's rows at d_D + r*(Np/P)*ldd, and
- * the pivot broadcast replaced by the shared pivot-row buffer.  d_D is the full Np x Np matrix
+/* The sharded schedule of apsp_reduced for `nranks` ranks, emulated in ONE process on the current
+ * device: every virtual rank gets its own owned-tile-row storage and runs the same kernels; the
+ * all-reduce of the pivot pieces is replaced by a shared pivot-row buffer (the pieces are disjoint)
+ * and the final gather by scattering every rank's upper tiles into d_D, the full Np x Np matrix
  * (Np = ear_plan_info(nranks).n_reduced_padded).  Used to test the multi-GPU path on one GPU; the
  * result must equal apsp_reduced bit for bit.  Asynchronous; errors as apsp_reduced. */
 ear_status_t apsp_reduced_emulated(ear_plan_t plan, int32_t nranks, int32_t *d_D, int64_t ldd,
                                    void *stream);
 
-/* All-gather the row blocks produced by apsp_reduced with `comm` into the full Np x Np matrix
- * d_D_full (ldd_full >= Np).  d_D_block may alias this rank's rows of d_D_full when
- * ldd_block == ldd_full and d_D_block == d_D_full + rank*(Np/P)*ldd_full. */
+/* Number of 128-row tile blocks a rank owns under the sharded layout of apsp_reduced (Np =
+ * ear_plan_info(nranks).n_reduced_padded).  Host-only. */
+int32_t ear_owned_tile_rows(int32_t n_reduced_padded, int32_t nranks, int32_t rank);
+
+/* Assemble the full Np x Np matrix d_D_full (ldd_full >= Np) from every rank's owned storage written
+ * by apsp_reduced with `comm`: each rank scatters its upper tiles and their mirrors into an
+ * INF-filled matrix, and one NCCL all-reduce(MIN) combines them.  d_D_block must not alias
+ * d_D_full.  Without comm, a plain copy. */
 ear_status_t ear_gather_reduced(ear_plan_t plan, const int32_t *d_D_block, int64_t ldd_block,
                                 int32_t *d_D_full, int64_t ldd_full, ear_comm_t comm, void *stream);
 

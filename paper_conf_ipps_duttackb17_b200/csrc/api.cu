@@ -1,6 +1,7 @@
 // C-ABI entry points of libearapsp.so (declared and documented in include/ear_apsp.h).
 #include <cstdarg>
 #include <cstring>
+#include <vector>
 
 #include "common.cuh"
 
@@ -159,18 +160,32 @@ ear_status_t apsp_reduced(ear_plan_t p, int32_t *d_D, int64_t ldd, ear_comm_t co
     return EAR_EINVAL;
   }
   cudaStream_t st = (cudaStream_t)stream;
-  if (p->flags & EAR_FLAG_SSSP) {   // rows by per-source SSSP: no inter-rank exchange in Phase II
-    const int32_t rows = Np / P, row0 = (comm ? comm->rank : 0) * rows;
-    return sssp_rows(p, d_D, ldd, Np, row0, rows, st);
-  }
   if (!comm) {
+    if (p->flags & EAR_FLAG_SSSP) return sssp_rows(p, d_D, ldd, Np, 0, Np, nullptr, st);
     EAR_TRY(fw_init_D(p, d_D, ldd, Np, 0, Np, st));
     return fw_single(d_D, ldd, Np, st);
   }
-  // with a communicator -- even one of a single rank -- the row-block schedule and its NCCL calls run
-  const int32_t rows = Np / P, row0 = comm->rank * rows;
-  EAR_TRY(fw_init_D(p, d_D, ldd, Np, row0, rows, st));
-  return fw_sharded(d_D, ldd, Np, comm, st);
+  // with a communicator -- even one of a single rank -- d_D holds this rank's owned tile rows
+  // (zig-zag assignment, ascending) and the sharded schedule with its NCCL calls runs
+  const int32_t nt = Np / TILE;
+  int32_t *d_rows = nullptr, nown = 0;
+  EAR_TRY(shard_rows_device(nt, P, comm->rank, &d_rows, &nown, st));
+  ear_status_t s = EAR_OK;
+  if (p->flags & EAR_FLAG_SSSP) {   // every rank its own rows: no exchange in Phase II
+    s = sssp_rows(p, d_D, ldd, Np, 0, nown * TILE, d_rows, st);
+  } else {
+    std::vector<int32_t> rows(nown);
+    if (nown > 0) {
+      cudaError_t e = cudaMemcpyAsync(rows.data(), d_rows, sizeof(int32_t) * nown, cudaMemcpyDeviceToHost, st);
+      if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+      if (e != cudaSuccess) { set_error("apsp_reduced: %s", cudaGetErrorString(e)); s = EAR_ECUDA; }
+    }
+    for (int32_t b = 0; b < nown && s == EAR_OK; ++b)
+      s = fw_init_D(p, d_D + (int64_t)b * TILE * ldd, ldd, Np, rows[b] * TILE, TILE, st);
+    if (s == EAR_OK) s = fw_sharded(d_D, ldd, Np, comm, st);
+  }
+  cudaFreeAsync(d_rows, st);
+  return s;
 }
 
 ear_status_t apsp_reduced_emulated(ear_plan_t p, int32_t nranks, int32_t *d_D, int64_t ldd, void *stream) {
@@ -181,9 +196,12 @@ ear_status_t apsp_reduced_emulated(ear_plan_t p, int32_t nranks, int32_t *d_D, i
     set_error("apsp_reduced_emulated: need ldd >= Np=%d, ldd %% 4 == 0, 16-byte aligned D", Np);
     return EAR_EINVAL;
   }
-  cudaStream_t st = (cudaStream_t)stream;
-  EAR_TRY(fw_init_D(p, d_D, ldd, Np, 0, Np, st));
-  return fw_sharded_emulated(d_D, ldd, Np, nranks, st);
+  return fw_sharded_emulated(p, d_D, ldd, Np, nranks, (cudaStream_t)stream);
+}
+
+int32_t ear_owned_tile_rows(int32_t n_reduced_padded, int32_t nranks, int32_t rank) {
+  if (nranks < 1 || rank < 0 || rank >= nranks) return 0;
+  return shard_nown(n_reduced_padded / TILE, nranks, rank);
 }
 
 ear_status_t ear_gather_reduced(ear_plan_t p, const int32_t *d_D_block, int64_t ldd_block, int32_t *d_D_full,
@@ -192,8 +210,6 @@ ear_status_t ear_gather_reduced(ear_plan_t p, const int32_t *d_D_block, int64_t 
   cudaStream_t st = (cudaStream_t)stream;
   const int32_t P = comm ? comm->nranks : 1;
   const int32_t Np = padded(p, P);
-  const int32_t rows = Np / P;
-  const int32_t rank = comm ? comm->rank : 0;
   if (ldd_block < Np || ldd_full < Np) { set_error("ear_gather_reduced: leading dimension < Np"); return EAR_EINVAL; }
   if (!comm) {
     if (d_D_block != d_D_full)
@@ -201,23 +217,7 @@ ear_status_t ear_gather_reduced(ear_plan_t p, const int32_t *d_D_block, int64_t 
                                      sizeof(int32_t) * Np, Np, cudaMemcpyDeviceToDevice, st));
     return EAR_OK;
   }
-  const int64_t cnt = (int64_t)rows * Np;
-  if (ldd_block == Np && ldd_full == Np) {
-    return comm_allgather(comm, d_D_block, d_D_full, cnt, st);
-  }
-  // general leading dimensions: pack, gather into a contiguous buffer, unpack
-  int32_t *tmp = nullptr;
-  EAR_CUDA_TRY(cudaMallocAsync((void **)&tmp, sizeof(int32_t) * (size_t)Np * Np, st));
-  EAR_CUDA_TRY(cudaMemcpy2DAsync(tmp + (int64_t)rank * cnt, sizeof(int32_t) * Np, d_D_block,
-                                 sizeof(int32_t) * ldd_block, sizeof(int32_t) * Np, rows, cudaMemcpyDeviceToDevice, st));
-  ear_status_t s = comm_allgather(comm, tmp + (int64_t)rank * cnt, tmp, cnt, st);
-  if (s == EAR_OK) {
-    cudaError_t e = cudaMemcpy2DAsync(d_D_full, sizeof(int32_t) * ldd_full, tmp, sizeof(int32_t) * Np,
-                                      sizeof(int32_t) * Np, Np, cudaMemcpyDeviceToDevice, st);
-    if (e != cudaSuccess) { set_error("gather unpack: %s", cudaGetErrorString(e)); s = EAR_ECUDA; }
-  }
-  cudaFreeAsync(tmp, st);
-  return s;
+  return fw_sharded_gather(d_D_block, ldd_block, Np, d_D_full, ldd_full, comm, st);
 }
 
 ear_status_t expand_ears(ear_plan_t p, const int32_t *d_D_full, int64_t ldd, int32_t row_begin, int32_t row_end,
@@ -254,10 +254,12 @@ static ear_status_t solve_rows(ear_plan_s *p, int32_t row_begin, int32_t row_end
     s = apsp_reduced(p, D, Np, nullptr, st);
     Dfull = D;
   } else {
+    const int32_t nown = shard_nown(Np / TILE, P, comm->rank);
     EAR_CUDA_TRY(cudaMallocAsync((void **)&Dfull, sizeof(int32_t) * (size_t)Np * Np, st));
-    D = Dfull + (int64_t)comm->rank * (Np / P) * Np;   // this rank's rows, in place
+    EAR_CUDA_TRY(cudaMallocAsync((void **)&D, sizeof(int32_t) * (size_t)std::max(nown, 1) * TILE * Np, st));
     s = apsp_reduced(p, D, Np, comm, st);
     if (s == EAR_OK) s = ear_gather_reduced(p, D, Np, Dfull, Np, comm, st);
+    cudaFreeAsync(D, st);
   }
   if (s == EAR_OK && d_out) s = expand_ears(p, Dfull, Np, row_begin, row_end, d_out, ldo, st);
   if (D_keep && s == EAR_OK) {

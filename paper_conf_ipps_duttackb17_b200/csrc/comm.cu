@@ -21,6 +21,11 @@ ear_status_t comm_bcast(ear_comm_s *comm, int32_t *buf, int64_t count, int32_t r
   return EAR_OK;
 }
 
+ear_status_t comm_allreduce_min(ear_comm_s *comm, int32_t *buf, int64_t count, cudaStream_t st) {
+  EAR_NCCL_TRY(ncclAllReduce(buf, buf, (size_t)count, ncclInt32, ncclMin, (ncclComm_t)comm->nccl, st));
+  return EAR_OK;
+}
+
 ear_status_t comm_allgather(ear_comm_s *comm, const int32_t *send, int32_t *recv, int64_t count,
                             cudaStream_t st) {
   EAR_NCCL_TRY(ncclAllGather(send, recv, (size_t)count, ncclInt32, (ncclComm_t)comm->nccl, st));

@@ -96,11 +96,21 @@ void plan_free(ear_plan_s *plan);
 ear_status_t fw_init_D(const ear_plan_s *plan, int32_t *D, int64_t ldd, int32_t Np, int32_t row0,
                        int32_t rows, cudaStream_t stream);
 ear_status_t fw_single(int32_t *D, int64_t ldd, int32_t Np, cudaStream_t stream);
-ear_status_t fw_sharded(int32_t *Dblk, int64_t ldd, int32_t Np, ear_comm_s *comm, cudaStream_t stream);
-ear_status_t fw_sharded_emulated(int32_t *D, int64_t ldd, int32_t Np, int32_t P, cudaStream_t stream);
+// row-block sharding: rank r owns the tile rows ti with (ti mod 2P) in {r, 2P-1-r} (zig-zag), stored
+// ascending as 128-row blocks
+ear_status_t fw_sharded(int32_t *S, int64_t ldd, int32_t Np, ear_comm_s *comm, cudaStream_t stream);
+ear_status_t fw_sharded_gather(const int32_t *S, int64_t ldd, int32_t Np, int32_t *Df, int64_t ldf, ear_comm_s *comm,
+                               cudaStream_t stream);
+ear_status_t fw_sharded_emulated(const ear_plan_s *plan, int32_t *D, int64_t ldd, int32_t Np, int32_t P,
+                                 cudaStream_t stream);
+int32_t shard_nown(int32_t nt, int32_t P, int32_t rank);
+ear_status_t shard_rows_device(int32_t nt, int32_t P, int32_t rank, int32_t **d_rows, int32_t *nown,
+                               cudaStream_t stream);
 // sssp.cu
+// rows [row0, row0+rows) of D, or -- with d_tile_rows -- the 128-row blocks listed there (local block b
+// holds global rows d_tile_rows[b]*128 ..), written consecutively into D
 ear_status_t sssp_rows(ear_plan_s *plan, int32_t *D, int64_t ldd, int32_t Np, int32_t row0, int32_t rows,
-                       cudaStream_t stream);
+                       const int32_t *d_tile_rows, cudaStream_t stream);
 // expand.cu
 ear_status_t expand(const ear_plan_s *plan, const int32_t *D, int64_t ldd, int32_t row_begin,
                     int32_t row_end, int32_t *out, int64_t ldo, cudaStream_t stream);
@@ -110,4 +120,5 @@ ear_status_t query_pairs(const ear_plan_s *plan, const int32_t *D, int64_t ldd, 
 ear_status_t comm_bcast(ear_comm_s *comm, int32_t *buf, int64_t count, int32_t root, cudaStream_t stream);
 ear_status_t comm_allgather(ear_comm_s *comm, const int32_t *send, int32_t *recv, int64_t count,
                             cudaStream_t stream);
+ear_status_t comm_allreduce_min(ear_comm_s *comm, int32_t *buf, int64_t count, cudaStream_t stream);
 }  // namespace ear

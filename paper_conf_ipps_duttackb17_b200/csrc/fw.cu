@@ -113,7 +113,7 @@ __global__ void __launch_bounds__(NT, 1) k_fw_phase1(int32_t *T, int64_t ldt) {
 // mbarriers (full: TMA bytes landed; empty: all 8 warps done reading), so no CTA-wide barrier sits
 // in the main loop and the next tile's first chunks are fetched while the current tile finishes.
 // Thread 0 doubles as the TMA producer.  The C tile lives in registers (8x8 per thread).
-enum { MODE_PIVOT_ROW = 0, MODE_UPPER = 1, MODE_ROWS = 2 };
+enum { MODE_PIVOT_ROW = 0, MODE_UPPER = 1, MODE_LIST = 2 };
 
 // Tile-kernel configuration: k-chunk depth, TMA ring depth, CTAs per SM, kk-loop unroll.
 template <int KC_, int ST_, int MINB_, int UNR_>
@@ -138,6 +138,12 @@ struct TileJob {
   int32_t mode;
   int32_t mirror;    // also write the transposed result into tile (tj, ti) (single GPU)
   int64_t ntiles;    // tiles in this launch
+  // MODE_LIST (row-block sharded): the rank's owned tile rows (ascending), the static prefix sums of
+  // their upper-tile counts (nt - ti), and per round k: mk = #owned rows < k, posk = position of row k
+  // in the owned list or -1
+  const int32_t *orow;
+  const int64_t *opre;
+  int32_t nown, mk, posk;
 };
 
 __device__ __forceinline__ uint32_t smem_u32(const void *p) { return (uint32_t)__cvta_generic_to_shared(p); }
@@ -174,12 +180,13 @@ __device__ __forceinline__ void tma_load_2d(void *dst, const CUtensorMap *map, i
       : "memory");
 }
 
-// decode the tile index into (ti, tj)
-__device__ __forceinline__ void decode_tile(const TileJob &J, int64_t idx, int &ti, int &tj) {
+// decode the tile index into (ti, tj) and the local tile row lr of C
+__device__ __forceinline__ void decode_tile(const TileJob &J, int64_t idx, int &ti, int &tj, int &lr) {
   const int k = J.k;
   if (J.mode == MODE_PIVOT_ROW) {
     ti = k;
     tj = (int)idx < k ? (int)idx : (int)idx + 1;
+    lr = ti - J.ti0;
     return;
   }
   if (J.mode == MODE_UPPER) {
@@ -194,14 +201,23 @@ __device__ __forceinline__ void decode_tile(const TileJob &J, int64_t idx, int &
     const int64_t b = a + (idx - (a * T - a * (a - 1) / 2));
     ti = (int)a < k ? (int)a : (int)a + 1;
     tj = (int)b < k ? (int)b : (int)b + 1;
+    lr = ti - J.ti0;
     return;
   }
-  // MODE_ROWS: local tile rows except the pivot row, all columns except the pivot column
-  const int64_t ncols = J.nt - 1;
-  int r = (int)(idx / ncols), cidx = (int)(idx % ncols);
-  ti = J.ti0 + r;
-  if (ti >= k && k >= J.ti0 && k < J.ti0 + J.nti) ti++;   // skip the pivot tile row if local
-  tj = cidx < k ? cidx : cidx + 1;
+  // MODE_LIST: the upper tiles (ti, tj >= ti) of the owned rows, without row k and column k.
+  // Per round, owned rows ti < k lose tile (ti, k) and row k (if owned) loses all its tiles.
+  auto pre = [&](int r) -> int64_t {
+    return J.opre[r] - min(r, J.mk) - ((J.posk >= 0 && r > J.posk) ? (int64_t)(J.nt - k) : 0);
+  };
+  int lo = 0, hi = J.nown - 1;   // largest r with pre(r) <= idx (ties: the last, skipping empty rows)
+  while (lo < hi) {
+    const int mid = (lo + hi + 1) >> 1;
+    if (pre(mid) <= idx) lo = mid; else hi = mid - 1;
+  }
+  lr = lo;
+  ti = J.orow[lo];
+  tj = ti + (int)(idx - pre(lo));
+  if (ti < k && tj >= k) ++tj;
 }
 
 template <class CF>
@@ -218,13 +234,15 @@ __global__ void __launch_bounds__(NT, CF::MINB) k_fw_tiles(const __grid_constant
   const int my_tiles = J.ntiles > (int64_t)blockIdx.x ? (int)((J.ntiles - 1 - blockIdx.x) / gridDim.x + 1) : 0;
   const int total_chunks = my_tiles * NCHUNK;
   int issued = 0;   // producer state (thread 0 only)
-  auto tile_of = [&](int it, int &ti, int &tj) { decode_tile(J, blockIdx.x + (int64_t)it * gridDim.x, ti, tj); };
+  auto tile_of = [&](int it, int &ti, int &tj, int &lr) {
+    decode_tile(J, blockIdx.x + (int64_t)it * gridDim.x, ti, tj, lr);
+  };
   auto produce = [&](int upto) {
     while (issued < upto) {
       const int st = issued % STAGES;
       if (issued >= STAGES) mbar_wait(&empty[st], (uint32_t)((issued / STAGES - 1) & 1));
-      int pti, ptj;
-      tile_of(issued / NCHUNK, pti, ptj);
+      int pti, ptj, plr;
+      tile_of(issued / NCHUNK, pti, ptj, plr);
       const int row = J.p_row0 + (issued % NCHUNK) * KC;
       mbar_arrive_tx(&full[st], 2 * SM_CHUNK * 4);
       tma_load_2d(sA + st * SM_CHUNK, &tmP, pti * TILE, row, &full[st]);
@@ -246,11 +264,11 @@ __global__ void __launch_bounds__(NT, CF::MINB) k_fw_tiles(const __grid_constant
 
   int g = 0;   // chunk counter (all threads)
   for (int it = 0; it < my_tiles; ++it) {
-    int ti, tj;
-    tile_of(it, ti, tj);
+    int ti, tj, lr;
+    tile_of(it, ti, tj, lr);
     int32_t c[8][8];
     // C tile straight from global memory into registers (its latency overlaps the in-flight TMA chunks)
-    int32_t *Ct = J.C + (int64_t)(ti - J.ti0) * TILE * J.ldc + (int64_t)tj * TILE;
+    int32_t *Ct = J.C + (int64_t)lr * TILE * J.ldc + (int64_t)tj * TILE;
 #pragma unroll
     for (int r = 0; r < 8; ++r) {
       const int i = (r < 4 ? 0 : 64) + ty * 4 + (r & 3);
@@ -301,21 +319,63 @@ __global__ void __launch_bounds__(NT, CF::MINB) k_fw_tiles(const __grid_constant
   }
 }
 
-// transposed copy of the pivot row block's slice into this rank's column tiles (i, k):
-// D[i-block rows][k-block cols] = P[0..128)[i-block]^T  (phase 2 columns by symmetry)
-__global__ void k_col_tiles_from_pivot(int32_t *C, int64_t ldc, const int32_t *P, int64_t ldp, int32_t k,
-                                       int32_t ti0, int32_t nti) {
+__global__ void k_fill(int32_t *p, int64_t n, int32_t v) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) p[i] = v;
+}
+
+// Pivot-row block <-> a rank's owned storage, round k (prow: 128 x Np, leading dimension Np).
+//   dir = 0 (gather):  prow[:, ti-block] = S(ti, k)^T for owned ti < k; prow[:, j >= k] = S(k, j) if row k owned
+//   dir = 1 (scatter): the inverse, after phases 1 and 2 updated prow
+// grid: (16 sub-blocks of 32 x 32, Np/128 column tiles, nown owned rows), 256 threads
+__global__ void k_prow_xfer(int32_t *S, int64_t ldd, const int32_t *orow, int32_t k, int32_t *prow, int32_t Np,
+                            int dir) {
   __shared__ int32_t t[32][33];
-  const int tile = blockIdx.y;                 // local tile row
-  const int ti = ti0 + tile;
-  if (ti == k) return;
-  const int bx = blockIdx.x & 3, by = blockIdx.x >> 2;  // 4 x 4 sub-blocks of 32 x 32
-  const int lx = threadIdx.x & 31, ly = threadIdx.x >> 5;  // 32 x 8
-  for (int yy = ly; yy < 32; yy += 8)   // P rows (k-local) by*32+yy, cols ti*128 + bx*32 + lx
-    t[yy][lx] = P[(int64_t)(by * 32 + yy) * ldp + (int64_t)ti * TILE + bx * 32 + lx];
+  const int lr = blockIdx.z, ti = orow[lr], tj = blockIdx.y;
+  const int bx = blockIdx.x & 3, by = blockIdx.x >> 2;         // 32 x 32 sub-block (bx: x, by: y)
+  const int lx = threadIdx.x & 31, ly = threadIdx.x >> 5;      // 32 x 8 threads
+  if (ti == k) {               // the pivot row's upper part: plain copy, tiles j >= k
+    if (tj < k) return;
+    for (int yy = ly; yy < 32; yy += 8) {
+      const int64_t row = by * 32 + yy, col = (int64_t)tj * TILE + bx * 32 + lx;
+      int32_t *s = S + ((int64_t)lr * TILE + row) * ldd + col;
+      int32_t *p = prow + row * Np + col;
+      if (dir == 0) *p = *s; else *s = *p;
+    }
+    return;
+  }
+  if (ti > k || tj != k) return;   // owned row below the pivot: its tile (ti, k) <-> prow[:, ti-block]^T
+  if (dir == 0) {
+    for (int yy = ly; yy < 32; yy += 8)   // S rows ti-block (bx*32+yy), cols k-block (by*32+lx)
+      t[yy][lx] = S[((int64_t)lr * TILE + bx * 32 + yy) * ldd + (int64_t)k * TILE + by * 32 + lx];
+    __syncthreads();
+    for (int yy = ly; yy < 32; yy += 8)   // prow rows (by*32+yy), cols ti-block (bx*32+lx)
+      prow[(int64_t)(by * 32 + yy) * Np + (int64_t)ti * TILE + bx * 32 + lx] = t[lx][yy];
+  } else {
+    for (int yy = ly; yy < 32; yy += 8)
+      t[yy][lx] = prow[(int64_t)(by * 32 + yy) * Np + (int64_t)ti * TILE + bx * 32 + lx];
+    __syncthreads();
+    for (int yy = ly; yy < 32; yy += 8)
+      S[((int64_t)lr * TILE + bx * 32 + yy) * ldd + (int64_t)k * TILE + by * 32 + lx] = t[lx][yy];
+  }
+}
+
+// owned upper tiles (ti, tj >= ti) -> full D, and their transposed mirrors (tj, ti)
+// grid: (16 sub-blocks, nt column tiles, nown owned rows), 256 threads
+__global__ void k_scatter_upper(const int32_t *S, int64_t ldd, const int32_t *orow, int32_t *Df, int64_t ldf) {
+  __shared__ int32_t t[32][33];
+  const int lr = blockIdx.z, ti = orow[lr], tj = blockIdx.y;
+  if (tj < ti) return;
+  const int bx = blockIdx.x & 3, by = blockIdx.x >> 2;
+  const int lx = threadIdx.x & 31, ly = threadIdx.x >> 5;
+  for (int yy = ly; yy < 32; yy += 8) {
+    const int32_t v = S[((int64_t)lr * TILE + by * 32 + yy) * ldd + (int64_t)tj * TILE + bx * 32 + lx];
+    Df[((int64_t)ti * TILE + by * 32 + yy) * ldf + (int64_t)tj * TILE + bx * 32 + lx] = v;
+    t[yy][lx] = v;
+  }
+  if (tj == ti) return;
   __syncthreads();
-  for (int yy = ly; yy < 32; yy += 8)   // C rows (tile-local) bx*32+yy, cols k*128 + by*32 + lx
-    C[(int64_t)(tile * TILE + bx * 32 + yy) * ldc + (int64_t)k * TILE + by * 32 + lx] = t[lx][yy];
+  for (int yy = ly; yy < 32; yy += 8)
+    Df[((int64_t)tj * TILE + bx * 32 + yy) * ldf + (int64_t)ti * TILE + by * 32 + lx] = t[lx][yy];
 }
 
 int g_num_sms = 0;
@@ -423,97 +483,216 @@ ear_status_t fw_single(int32_t *D, int64_t ldd, int32_t Np, cudaStream_t st) {
   return EAR_OK;
 }
 
-// Row-block sharded FW.  Rank r holds rows [r*R, (r+1)*R) of D (R = Np / P, a multiple of 128).
-// Round k: the owner of pivot block k closes the pivot tile and its pivot-row tiles and copies the
-// 128 x Np pivot row block into `prow`; the block reaches every rank (NCCL broadcast, or the same
-// buffer when emulated); every rank fills its pivot-column tiles by symmetry and updates its other
-// tiles with both operands taken from `prow`.
-struct ShardCtx {
-  int32_t *Dblk;    // this rank's row block
-  int64_t ldd;
-  int32_t Np, nt, P, rank, nti, ti0;
-  int32_t *prow;    // 128 x Np pivot row block (leading dimension Np)
-  CUtensorMap map_blk, map_prow;
+// ---------------------------------------------------------------------------- row-block sharding
+// Symmetric row-block sharding.  Tile rows are dealt to ranks in a zig-zag (rows r and 2P-1-r of every
+// group of 2P), so the UPPER tiles (ti, tj >= ti) -- the only authoritative ones -- balance across
+// ranks; rank r stores its owned tile rows (ascending) as 128-row blocks.  Round k:
+//   1. every rank writes its pieces of the pivot row block into prow (tile (k, j >= k) from the owner
+//      of row k, tiles (i < k, k) transposed from the owners of rows i), INF elsewhere, and an
+//      all-reduce(MIN) over NCCL assembles the block on every rank;
+//   2. every rank closes the pivot tile (phase 1) and updates the pivot row block (phase 2) locally;
+//   3. owners copy the updated pivot pieces back into their storage;
+//   4. every rank updates its owned upper tiles outside row/column k (phase 3), both operands from prow.
+// Per-rank min-plus work is (N_r^3 / 2) / P + the redundant phase 1/2, i.e. the single-GPU symmetric
+// halving survives the sharding.  The final D is assembled by scattering every rank's upper tiles and
+// their mirrors into an INF-filled full matrix and one all-reduce(MIN).
+
+std::vector<int32_t> shard_rows(int32_t nt, int32_t P, int32_t rank) {
+  std::vector<int32_t> rows;
+  for (int32_t ti = 0; ti < nt; ++ti) {
+    const int32_t o = ti % (2 * P);
+    if ((o < P ? o : 2 * P - 1 - o) == rank) rows.push_back(ti);
+  }
+  return rows;
+}
+
+struct Shard {
+  int32_t *S = nullptr;        // owned storage: nown x 128 rows x ldd
+  int64_t ldd = 0;
+  int32_t Np = 0, nt = 0, P = 1, rank = 0, nown = 0;
+  std::vector<int32_t> rows;
+  int32_t *d_rows = nullptr;
+  int64_t *d_pre = nullptr;
 };
 
-static ear_status_t shard_ctx(ShardCtx *c, int32_t *Dblk, int64_t ldd, int32_t Np, int32_t P, int32_t rank,
-                              int32_t *prow) {
-  c->Dblk = Dblk; c->ldd = ldd; c->Np = Np; c->nt = Np / TILE; c->P = P; c->rank = rank;
-  c->nti = c->nt / P; c->ti0 = rank * c->nti; c->prow = prow;
-  EAR_TRY(make_map(&c->map_blk, Dblk, (int64_t)c->nti * TILE, Np, ldd, fw_kc()));
-  EAR_TRY(make_map(&c->map_prow, prow, TILE, Np, Np, fw_kc()));
+static ear_status_t shard_setup(Shard *sh, int32_t *S, int64_t ldd, int32_t Np, int32_t P, int32_t rank,
+                                cudaStream_t st) {
+  sh->S = S; sh->ldd = ldd; sh->Np = Np; sh->nt = Np / TILE; sh->P = P; sh->rank = rank;
+  sh->rows = shard_rows(sh->nt, P, rank);
+  sh->nown = (int32_t)sh->rows.size();
+  std::vector<int64_t> pre(sh->nown + 1, 0);
+  for (int32_t r = 0; r < sh->nown; ++r) pre[r + 1] = pre[r] + (sh->nt - sh->rows[r]);
+  const size_t nr = std::max<int32_t>(sh->nown, 1);
+  EAR_CUDA_TRY(cudaMallocAsync((void **)&sh->d_rows, sizeof(int32_t) * nr, st));
+  EAR_CUDA_TRY(cudaMallocAsync((void **)&sh->d_pre, sizeof(int64_t) * (nr + 1), st));
+  if (sh->nown > 0) {
+    EAR_CUDA_TRY(cudaMemcpyAsync(sh->d_rows, sh->rows.data(), sizeof(int32_t) * sh->nown, cudaMemcpyHostToDevice, st));
+    EAR_CUDA_TRY(cudaMemcpyAsync(sh->d_pre, pre.data(), sizeof(int64_t) * (sh->nown + 1), cudaMemcpyHostToDevice, st));
+    EAR_CUDA_TRY(cudaStreamSynchronize(st));   // host vectors are about to go out of scope
+  }
   return EAR_OK;
 }
 
-static ear_status_t shard_owner_step(const ShardCtx &c, int k, cudaStream_t st) {
+static void shard_free(Shard *sh, cudaStream_t st) {
+  if (sh->d_rows) cudaFreeAsync(sh->d_rows, st);
+  if (sh->d_pre) cudaFreeAsync(sh->d_pre, st);
+  sh->d_rows = nullptr; sh->d_pre = nullptr;
+}
+
+static ear_status_t fill(int32_t *p, int64_t n, int32_t v, cudaStream_t st) {
+  if (n <= 0) return EAR_OK;
+  EAR_LAUNCH(k_fill, (int)std::min<int64_t>(ceil_div(n, 256), 148 * 16), 256, 0, st)(p, n, v);
+  return EAR_OK;
+}
+
+static ear_status_t shard_xfer(const Shard &sh, int k, int32_t *prow, int dir, cudaStream_t st) {
+  if (sh.nown == 0) return EAR_OK;
+  dim3 g(16, sh.nt, sh.nown);
+  EAR_LAUNCH(k_prow_xfer, g, 256, 0, st)(sh.S, sh.ldd, sh.d_rows, k, prow, sh.Np, dir);
+  return EAR_OK;
+}
+
+// phases 1 and 2 on the assembled pivot row block
+static ear_status_t shard_pivot(int32_t *prow, const CUtensorMap &map_prow, int32_t Np, int k, cudaStream_t st) {
+  const int nt = Np / TILE;
   const double tile_ops = (double)TILE * TILE * TILE;
-  int32_t *Pk = c.Dblk + (int64_t)(k - c.ti0) * TILE * c.ldd;
   int s1 = prof_begin(PK_FW_P1, st);
-  EAR_LAUNCH(k_fw_phase1, 1, NT, 0, st)(Pk + (int64_t)k * TILE, c.ldd);
+  EAR_LAUNCH(k_fw_phase1, 1, NT, 0, st)(prow + (int64_t)k * TILE, Np);
   prof_end(s1, st, tile_ops);
-  // pivot-row tiles; C rows are the pivot rows themselves (ti0 = k: local row offset 0)
-  // pivot-row tiles (ti = k inside this rank's block)
-  TileJob J{c.Dblk, c.ldd, (k - c.ti0) * TILE, k, c.nt, c.ti0, c.nti, MODE_PIVOT_ROW, 0, 0};
+  TileJob J{prow, Np, 0, k, nt, k, 1, MODE_PIVOT_ROW, 0, 0, nullptr, nullptr, 0, 0, -1};
   int s2 = prof_begin(PK_FW_P2, st);
-  EAR_TRY(launch_tiles(c.map_blk, J, c.nt - 1, st));
-  prof_end(s2, st, (c.nt - 1) * tile_ops);
-  EAR_CUDA_TRY(cudaMemcpy2DAsync(c.prow, sizeof(int32_t) * c.Np, Pk, sizeof(int32_t) * c.ldd,
-                                 sizeof(int32_t) * c.Np, TILE, cudaMemcpyDeviceToDevice, st));
+  EAR_TRY(launch_tiles(map_prow, J, nt - 1, st));
+  prof_end(s2, st, (nt - 1) * tile_ops);
   return EAR_OK;
 }
 
-static ear_status_t shard_update_step(const ShardCtx &c, int k, cudaStream_t st) {
-  const double tile_ops = (double)TILE * TILE * TILE;
-  const int owner = k / c.nti;
-  dim3 g(16, c.nti);
-  EAR_LAUNCH(k_col_tiles_from_pivot, g, 256, 0, st)(c.Dblk, c.ldd, c.prow, c.Np, k, c.ti0, c.nti);
-  const int rows_here = (owner == c.rank) ? c.nti - 1 : c.nti;
-  TileJob J{c.Dblk, c.ldd, 0, k, c.nt, c.ti0, c.nti, MODE_ROWS, 0, 0};
+static ear_status_t shard_phase3(const Shard &sh, const CUtensorMap &map_prow, int k, cudaStream_t st) {
+  int mk = 0, posk = -1;
+  for (int32_t r = 0; r < sh.nown; ++r) {
+    if (sh.rows[r] < k) ++mk;
+    if (sh.rows[r] == k) posk = r;
+  }
+  int64_t total = 0;
+  for (int32_t r = 0; r < sh.nown; ++r) {
+    const int32_t ti = sh.rows[r];
+    total += ti == k ? 0 : (sh.nt - ti) - (ti < k ? 1 : 0);
+  }
+  TileJob J{sh.S, sh.ldd, 0, k, sh.nt, 0, sh.nown, MODE_LIST, 0, 0, sh.d_rows, sh.d_pre, sh.nown, mk, posk};
   int s3 = prof_begin(PK_FW_P3, st);
-  EAR_TRY(launch_tiles(c.map_prow, J, (int64_t)rows_here * (c.nt - 1), st));
-  prof_end(s3, st, (double)rows_here * (c.nt - 1) * tile_ops);
+  EAR_TRY(launch_tiles(map_prow, J, total, st));
+  prof_end(s3, st, (double)total * TILE * TILE * TILE);
   return EAR_OK;
 }
 
-ear_status_t fw_sharded(int32_t *Dblk, int64_t ldd, int32_t Np, ear_comm_s *comm, cudaStream_t st) {
+ear_status_t fw_sharded(int32_t *S, int64_t ldd, int32_t Np, ear_comm_s *comm, cudaStream_t st) {
+  Shard sh;
+  EAR_TRY(shard_setup(&sh, S, ldd, Np, comm->nranks, comm->rank, st));
   int32_t *prow = nullptr;
   EAR_CUDA_TRY(cudaMallocAsync((void **)&prow, sizeof(int32_t) * (size_t)TILE * Np, st));
-  ShardCtx c;
-  ear_status_t status = shard_ctx(&c, Dblk, ldd, Np, comm->nranks, comm->rank, prow);
-  for (int k = 0; k < c.nt && status == EAR_OK; ++k) {
-    const int owner = k / c.nti;
-    if (owner == c.rank) status = shard_owner_step(c, k, st);
-    if (status != EAR_OK) break;
-    int sc = prof_begin(PK_COMM, st);
-    status = comm_bcast(comm, prow, (int64_t)TILE * Np, owner, st);
-    prof_end(sc, st, 0);
-    if (status != EAR_OK) break;
-    status = shard_update_step(c, k, st);
+  CUtensorMap map_prow;
+  ear_status_t status = make_map(&map_prow, prow, TILE, Np, Np, fw_kc());
+  for (int k = 0; k < sh.nt && status == EAR_OK; ++k) {
+    status = fill(prow, (int64_t)TILE * Np, INF, st);
+    if (status == EAR_OK) status = shard_xfer(sh, k, prow, 0, st);
+    if (status == EAR_OK) {
+      int sc = prof_begin(PK_COMM, st);
+      status = comm_allreduce_min(comm, prow, (int64_t)TILE * Np, st);
+      prof_end(sc, st, 0);
+    }
+    if (status == EAR_OK) status = shard_pivot(prow, map_prow, Np, k, st);
+    if (status == EAR_OK) status = shard_xfer(sh, k, prow, 1, st);
+    if (status == EAR_OK) status = shard_phase3(sh, map_prow, k, st);
   }
   cudaFreeAsync(prow, st);
+  shard_free(&sh, st);
   if (status != EAR_OK) return status;
   EAR_CUDA_TRY(cudaGetLastError());
   return EAR_OK;
 }
 
-// The same schedule for P ranks emulated in one process on one device (tests of the multi-GPU
-// path on a single GPU): D is the full matrix, rank r's block starts at row r*Np/P, and the
-// broadcast is the shared pivot-row buffer itself.
-ear_status_t fw_sharded_emulated(int32_t *D, int64_t ldd, int32_t Np, int32_t P, cudaStream_t st) {
-  int32_t *prow = nullptr;
-  EAR_CUDA_TRY(cudaMallocAsync((void **)&prow, sizeof(int32_t) * (size_t)TILE * Np, st));
-  const int32_t R = Np / P;
+// Full D from every rank's owned upper tiles (INF fill + scatter + all-reduce MIN).
+ear_status_t fw_sharded_gather(const int32_t *S, int64_t ldd, int32_t Np, int32_t *Df, int64_t ldf, ear_comm_s *comm,
+                               cudaStream_t st) {
+  Shard sh;
+  EAR_TRY(shard_setup(&sh, const_cast<int32_t *>(S), ldd, Np, comm->nranks, comm->rank, st));
   ear_status_t status = EAR_OK;
-  const int nt = Np / TILE, nti = nt / P;
-  std::vector<ShardCtx> ctx(P);
-  for (int r = 0; r < P && status == EAR_OK; ++r)
-    status = shard_ctx(&ctx[r], D + (int64_t)r * R * ldd, ldd, Np, P, r, prow);
-  for (int k = 0; k < nt && status == EAR_OK; ++k) {
-    const int owner = k / nti;
-    status = shard_owner_step(ctx[owner], k, st);
-    for (int r = 0; r < P && status == EAR_OK; ++r) status = shard_update_step(ctx[r], k, st);
+  if (ldf == Np) {
+    status = fill(Df, (int64_t)Np * Np, INF, st);
+  } else {
+    for (int32_t r = 0; r < Np && status == EAR_OK; ++r) status = fill(Df + (int64_t)r * ldf, Np, INF, st);
   }
-  cudaFreeAsync(prow, st);
+  if (status == EAR_OK && sh.nown > 0) {
+    dim3 g(16, sh.nt, sh.nown);
+    EAR_LAUNCH(k_scatter_upper, g, 256, 0, st)(sh.S, sh.ldd, sh.d_rows, Df, ldf);
+  }
+  if (status == EAR_OK) {
+    int sc = prof_begin(PK_COMM, st);
+    if (ldf == Np) {
+      status = comm_allreduce_min(comm, Df, (int64_t)Np * Np, st);
+    } else {
+      for (int32_t r = 0; r < Np && status == EAR_OK; ++r) status = comm_allreduce_min(comm, Df + (int64_t)r * ldf, Np, st);
+    }
+    prof_end(sc, st, 0);
+  }
+  shard_free(&sh, st);
+  if (status != EAR_OK) return status;
+  EAR_CUDA_TRY(cudaGetLastError());
+  return EAR_OK;
+}
+
+int32_t shard_nown(int32_t nt, int32_t P, int32_t rank) { return (int32_t)shard_rows(nt, P, rank).size(); }
+
+ear_status_t shard_rows_device(int32_t nt, int32_t P, int32_t rank, int32_t **d_rows, int32_t *nown, cudaStream_t st) {
+  std::vector<int32_t> rows = shard_rows(nt, P, rank);
+  *nown = (int32_t)rows.size();
+  EAR_CUDA_TRY(cudaMallocAsync((void **)d_rows, sizeof(int32_t) * std::max<size_t>(rows.size(), 1), st));
+  if (!rows.empty()) {
+    EAR_CUDA_TRY(cudaMemcpyAsync(*d_rows, rows.data(), sizeof(int32_t) * rows.size(), cudaMemcpyHostToDevice, st));
+    EAR_CUDA_TRY(cudaStreamSynchronize(st));
+  }
+  return EAR_OK;
+}
+
+// The same schedule for P ranks emulated in one process on one device (tests of the multi-GPU path on
+// one GPU): every virtual rank has its own owned storage, the shared prow stands in for the
+// all-reduce (the ranks' pieces are disjoint), and the ranks' upper tiles are scattered into D.
+ear_status_t fw_sharded_emulated(const ear_plan_s *plan, int32_t *D, int64_t ldd, int32_t Np, int32_t P,
+                                 cudaStream_t st) {
+  const int nt = Np / TILE;
+  std::vector<Shard> sh(P);
+  ear_status_t status = EAR_OK;
+  for (int r = 0; r < P && status == EAR_OK; ++r) {
+    const size_t nown = shard_rows(nt, P, r).size();
+    int32_t *S = nullptr;
+    EAR_CUDA_TRY(cudaMallocAsync((void **)&S, sizeof(int32_t) * std::max<size_t>(nown, 1) * TILE * Np, st));
+    status = shard_setup(&sh[r], S, Np, Np, P, r, st);
+    for (int32_t lr = 0; lr < sh[r].nown && status == EAR_OK; ++lr)
+      status = fw_init_D(plan, S + (int64_t)lr * TILE * Np, Np, Np, sh[r].rows[lr] * TILE, TILE, st);
+  }
+  int32_t *prow = nullptr;
+  if (status == EAR_OK) {
+    cudaError_t e = cudaMallocAsync((void **)&prow, sizeof(int32_t) * (size_t)TILE * Np, st);
+    if (e != cudaSuccess) { set_error("emulated prow: %s", cudaGetErrorString(e)); status = EAR_ENOMEM; }
+  }
+  CUtensorMap map_prow;
+  if (status == EAR_OK) status = make_map(&map_prow, prow, TILE, Np, Np, fw_kc());
+  for (int k = 0; k < nt && status == EAR_OK; ++k) {
+    status = fill(prow, (int64_t)TILE * Np, INF, st);
+    for (int r = 0; r < P && status == EAR_OK; ++r) status = shard_xfer(sh[r], k, prow, 0, st);
+    if (status == EAR_OK) status = shard_pivot(prow, map_prow, Np, k, st);
+    for (int r = 0; r < P && status == EAR_OK; ++r) status = shard_xfer(sh[r], k, prow, 1, st);
+    for (int r = 0; r < P && status == EAR_OK; ++r) status = shard_phase3(sh[r], map_prow, k, st);
+  }
+  for (int r = 0; r < P && status == EAR_OK; ++r) {
+    if (sh[r].nown == 0) continue;
+    dim3 g(16, nt, sh[r].nown);
+    EAR_LAUNCH(k_scatter_upper, g, 256, 0, st)(sh[r].S, sh[r].ldd, sh[r].d_rows, D, ldd);
+  }
+  if (prow) cudaFreeAsync(prow, st);
+  for (int r = 0; r < P; ++r) {
+    if (sh[r].S) cudaFreeAsync(sh[r].S, st);
+    shard_free(&sh[r], st);
+  }
   if (status != EAR_OK) return status;
   EAR_CUDA_TRY(cudaGetLastError());
   return EAR_OK;

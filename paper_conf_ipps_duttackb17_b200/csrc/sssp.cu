@@ -42,18 +42,19 @@ __global__ void k_r_split(const uint64_t *keys, int64_t A, int32_t *col, int32_t
 
 __device__ __forceinline__ int32_t ld_cg(const int32_t *p) { return __ldcg(p); }
 
-// rows [src0, src1) of D (global rows; this launch writes D + (src - row0) * ldd)
+// sources: src0 + li, or (with trows) trows[li / 128] * 128 + li % 128; row li of D receives source li
 __global__ void __launch_bounds__(NT) k_sssp_bf(const int32_t *__restrict__ rowptr, const int32_t *__restrict__ col,
                                                const int32_t *__restrict__ wt, int32_t nr, int32_t Np, int32_t *D,
-                                               int64_t ldd, int32_t row0, int32_t src0, int32_t src1,
+                                               int64_t ldd, int32_t src0, int32_t nsrc, const int32_t *trows,
                                                unsigned long long *stats) {
   extern __shared__ uint32_t bits[];        // [2][W] frontier bitmaps
   __shared__ int flag[3];
   const int W = (Np + 31) >> 5;
   const int tid = threadIdx.x;
   unsigned long long my_rounds = 0, my_relax = 0, my_improve = 0, my_visits = 0;
-  for (int32_t src = src0 + blockIdx.x; src < src1; src += gridDim.x) {
-    int32_t *dist = D + (int64_t)(src - row0) * ldd;
+  for (int32_t li = blockIdx.x; li < nsrc; li += gridDim.x) {
+    const int32_t src = trows ? trows[li >> 7] * TILE + (li & (TILE - 1)) : src0 + li;
+    int32_t *dist = D + (int64_t)li * ldd;
     for (int i = tid * 4; i < Np; i += NT * 4)   // Np % 4 == 0, ldd % 4 == 0
       *reinterpret_cast<int4 *>(dist + i) = make_int4(INF, INF, INF, INF);
     for (int w = tid; w < 2 * W; w += NT) bits[w] = 0u;
@@ -119,8 +120,9 @@ constexpr int SSSP_LIST = 4096;   // frontier list capacity per pass
 
 template <int NTS, int K>
 __global__ void __launch_bounds__(NTS) k_sssp_smem(const int32_t *__restrict__ rowptr, const int2 *__restrict__ arcs,
-                                                   int32_t nr, int32_t Np, int32_t *D, int64_t ldd, int32_t row0,
-                                                   int32_t src0, int32_t src1, unsigned long long *stats) {
+                                                   int32_t nr, int32_t Np, int32_t *D, int64_t ldd,
+                                                   int32_t src0, int32_t nsrc, const int32_t *trows,
+                                                   unsigned long long *stats) {
   extern __shared__ __align__(16) int32_t sm[];
   int32_t *dist = sm;                                                 // [Np]
   int32_t *list = sm + Np;                                            // [SSSP_LIST]
@@ -131,7 +133,8 @@ __global__ void __launch_bounds__(NTS) k_sssp_smem(const int32_t *__restrict__ r
   const int KW = (W + NTS - 1) / NTS;       // bitmap words per thread (contiguous)
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   unsigned long long my_rounds = 0, my_relax = 0;
-  for (int32_t src = src0 + blockIdx.x; src < src1; src += gridDim.x) {
+  for (int32_t li = blockIdx.x; li < nsrc; li += gridDim.x) {
+    const int32_t src = trows ? trows[li >> 7] * TILE + (li & (TILE - 1)) : src0 + li;
     for (int i = tid; i < Np; i += NTS) dist[i] = INF;
     for (int w = tid; w < 2 * W; w += NTS) bits[w] = 0u;
     if (tid < 3) flag[tid] = 0;
@@ -257,7 +260,7 @@ __global__ void __launch_bounds__(NTS) k_sssp_smem(const int32_t *__restrict__ r
       }
     }
     __syncthreads();
-    int32_t *row = D + (int64_t)(src - row0) * ldd;
+    int32_t *row = D + (int64_t)li * ldd;
     for (int i = tid * 4; i < Np; i += NTS * 4)   // Np % 4 == 0, 16-byte aligned rows
       *reinterpret_cast<int4 *>(row + i) = *reinterpret_cast<const int4 *>(dist + i);
     __syncthreads();
@@ -275,7 +278,7 @@ __global__ void __launch_bounds__(NTS) k_sssp_smem(const int32_t *__restrict__ r
 // round's appends exceed the list capacity, the next round falls back to scanning its bitmap.
 template <int NTS, int K>
 __global__ void __launch_bounds__(NTS) k_sssp_list(const int2 *__restrict__ ell, int32_t nr, int32_t Np, int32_t *D,
-                                                   int64_t ldd, int32_t row0, int32_t src0, int32_t src1, int cap,
+                                                   int64_t ldd, int32_t src0, int32_t nsrc, const int32_t *trows, int cap,
                                                    unsigned long long *stats) {
   extern __shared__ __align__(16) int32_t sm[];
   const int W = (Np + 31) >> 5;
@@ -287,7 +290,8 @@ __global__ void __launch_bounds__(NTS) k_sssp_list(const int2 *__restrict__ ell,
   __shared__ int cnt[3], ovf[3];
   const int tid = threadIdx.x;
   unsigned long long my_rounds = 0, my_relax = 0;
-  for (int32_t src = src0 + blockIdx.x; src < src1; src += gridDim.x) {
+  for (int32_t li = blockIdx.x; li < nsrc; li += gridDim.x) {
+    const int32_t src = trows ? trows[li >> 7] * TILE + (li & (TILE - 1)) : src0 + li;
     for (int i = tid; i < Np; i += NTS) dist[i] = INF;
     for (int w = tid; w < 2 * W; w += NTS) M0[w] = 0u;
     if (tid < 3) { cnt[tid] = 0; ovf[tid] = 0; }
@@ -370,7 +374,7 @@ __global__ void __launch_bounds__(NTS) k_sssp_list(const int2 *__restrict__ ell,
       }
     }
     __syncthreads();
-    int32_t *row = D + (int64_t)(src - row0) * ldd;
+    int32_t *row = D + (int64_t)li * ldd;
     for (int i = tid * 4; i < Np; i += NTS * 4)   // Np % 4 == 0, 16-byte aligned rows
       *reinterpret_cast<int4 *>(row + i) = *reinterpret_cast<const int4 *>(dist + i);
     __syncthreads();
@@ -463,6 +467,7 @@ ear_status_t sssp_prepare(ear_plan_s *p, cudaStream_t st) {
 
 template <int NTS, int K>
 static ear_status_t sssp_launch(ear_plan_s *p, int32_t *D, int64_t ldd, int32_t Np, int32_t row0, int32_t rows,
+                                const int32_t *trows,
                                 int smem_s, int nsm, unsigned long long *d_stats, cudaStream_t st) {
   static int attr_s = 0;
   if (smem_s > attr_s) {
@@ -474,7 +479,7 @@ static ear_status_t sssp_launch(ear_plan_s *p, int32_t *D, int64_t ldd, int32_t 
   const int64_t grid = std::min<int64_t>(rows, (int64_t)nsm * std::max(per_sm, 1));
   int s = prof_begin(PK_SSSP, st);
   EAR_LAUNCH((k_sssp_smem<NTS, K>), (unsigned)grid, NTS, smem_s, st)(
-      p->r_rowptr, reinterpret_cast<const int2 *>(p->r_arcs), p->n_reduced, Np, D, ldd, row0, row0, row0 + rows,
+      p->r_rowptr, reinterpret_cast<const int2 *>(p->r_arcs), p->n_reduced, Np, D, ldd, row0, rows, trows,
       d_stats);
   prof_end(s, st, (double)rows * (double)p->n_rarcs);
   if (d_stats) {
@@ -490,6 +495,7 @@ static ear_status_t sssp_launch(ear_plan_s *p, int32_t *D, int64_t ldd, int32_t 
 
 template <int NTS, int K>
 static ear_status_t sssp_list_launch(ear_plan_s *p, int32_t *D, int64_t ldd, int32_t Np, int32_t row0, int32_t rows,
+                                     const int32_t *trows,
                                      int max_smem, int nsm, unsigned long long *d_stats, cudaStream_t st) {
   const int W = (Np + 31) / 32;
   const int fixed = 4 * Np + 8 * W + 64;
@@ -505,7 +511,7 @@ static ear_status_t sssp_list_launch(ear_plan_s *p, int32_t *D, int64_t ldd, int
   const int64_t grid = std::min<int64_t>(rows, (int64_t)nsm * std::max(per_sm, 1));
   int s = prof_begin(PK_SSSP, st);
   EAR_LAUNCH((k_sssp_list<NTS, K>), (unsigned)grid, NTS, smem, st)(
-      reinterpret_cast<const int2 *>(p->r_arcs), p->n_reduced, Np, D, ldd, row0, row0, row0 + rows, cap, d_stats);
+      reinterpret_cast<const int2 *>(p->r_arcs), p->n_reduced, Np, D, ldd, row0, rows, trows, cap, d_stats);
   prof_end(s, st, (double)rows * (double)p->n_rarcs);
   if (d_stats) {
     unsigned long long h[4];
@@ -520,6 +526,7 @@ static ear_status_t sssp_list_launch(ear_plan_s *p, int32_t *D, int64_t ldd, int
 
 // Rows [row0, row0 + rows) of D (row-major, ldd) by per-source Bellman-Ford on G^r.
 ear_status_t sssp_rows(ear_plan_s *p, int32_t *D, int64_t ldd, int32_t Np, int32_t row0, int32_t rows,
+                       const int32_t *trows,
                        cudaStream_t st) {
   EAR_TRY(sssp_prepare(p, st));
   if (rows <= 0) return EAR_OK;
@@ -563,19 +570,19 @@ ear_status_t sssp_rows(ear_plan_s *p, int32_t *D, int64_t ldd, int32_t Np, int32
     const int list_smem = 4 * Np + 8 * std::min(Np, (max_smem - (4 * Np + 8 * W + 64)) / 8) + 8 * W;
     if (2 * list_smem + 2048 <= max_smem + 1024) {
       switch (p->r_ell_k) {
-        case 4: return sssp_list_launch<NTS, 4>(p, D, ldd, Np, row0, rows, max_smem, nsm, want_stats ? d_stats : nullptr, st);
-        case 8: return sssp_list_launch<NTS, 8>(p, D, ldd, Np, row0, rows, max_smem, nsm, want_stats ? d_stats : nullptr, st);
-        case 12: return sssp_list_launch<NTS, 12>(p, D, ldd, Np, row0, rows, max_smem, nsm, want_stats ? d_stats : nullptr, st);
-        case 16: return sssp_list_launch<NTS, 16>(p, D, ldd, Np, row0, rows, max_smem, nsm, want_stats ? d_stats : nullptr, st);
+        case 4: return sssp_list_launch<NTS, 4>(p, D, ldd, Np, row0, rows, trows, max_smem, nsm, want_stats ? d_stats : nullptr, st);
+        case 8: return sssp_list_launch<NTS, 8>(p, D, ldd, Np, row0, rows, trows, max_smem, nsm, want_stats ? d_stats : nullptr, st);
+        case 12: return sssp_list_launch<NTS, 12>(p, D, ldd, Np, row0, rows, trows, max_smem, nsm, want_stats ? d_stats : nullptr, st);
+        case 16: return sssp_list_launch<NTS, 16>(p, D, ldd, Np, row0, rows, trows, max_smem, nsm, want_stats ? d_stats : nullptr, st);
         default: break;
       }
     }
     switch (p->r_ell_k) {
-      case 4: return sssp_launch<NTS, 4>(p, D, ldd, Np, row0, rows, smem_s, nsm, want_stats ? d_stats : nullptr, st);
-      case 8: return sssp_launch<NTS, 8>(p, D, ldd, Np, row0, rows, smem_s, nsm, want_stats ? d_stats : nullptr, st);
-      case 12: return sssp_launch<NTS, 12>(p, D, ldd, Np, row0, rows, smem_s, nsm, want_stats ? d_stats : nullptr, st);
-      case 16: return sssp_launch<NTS, 16>(p, D, ldd, Np, row0, rows, smem_s, nsm, want_stats ? d_stats : nullptr, st);
-      default: return sssp_launch<NTS, 0>(p, D, ldd, Np, row0, rows, smem_s, nsm, want_stats ? d_stats : nullptr, st);
+      case 4: return sssp_launch<NTS, 4>(p, D, ldd, Np, row0, rows, trows, smem_s, nsm, want_stats ? d_stats : nullptr, st);
+      case 8: return sssp_launch<NTS, 8>(p, D, ldd, Np, row0, rows, trows, smem_s, nsm, want_stats ? d_stats : nullptr, st);
+      case 12: return sssp_launch<NTS, 12>(p, D, ldd, Np, row0, rows, trows, smem_s, nsm, want_stats ? d_stats : nullptr, st);
+      case 16: return sssp_launch<NTS, 16>(p, D, ldd, Np, row0, rows, trows, smem_s, nsm, want_stats ? d_stats : nullptr, st);
+      default: return sssp_launch<NTS, 0>(p, D, ldd, Np, row0, rows, trows, smem_s, nsm, want_stats ? d_stats : nullptr, st);
     }
   }
   const int smem = 2 * W * 4;
@@ -591,7 +598,7 @@ ear_status_t sssp_rows(ear_plan_s *p, int32_t *D, int64_t ldd, int32_t Np, int32
   const int64_t grid = std::min<int64_t>({(int64_t)rows, (int64_t)nsm * std::max(per_sm, 1), l2_rows});
   int s = prof_begin(PK_SSSP, st);
   EAR_LAUNCH(k_sssp_bf, (unsigned)grid, NT, smem, st)(p->r_rowptr, p->r_col, p->r_w, p->n_reduced, Np, D, ldd, row0,
-                                                      row0, row0 + rows, want_stats ? d_stats : nullptr);
+                                                      rows, trows, want_stats ? d_stats : nullptr);
   if (want_stats) {
     unsigned long long h[4];
     EAR_CUDA_TRY(cudaMemcpyAsync(h, d_stats, 32, cudaMemcpyDeviceToHost, st));

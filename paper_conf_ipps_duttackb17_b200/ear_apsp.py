@@ -63,6 +63,7 @@ SIGNATURES = {
     "ear_plan_destroy": (None, [_P]),
     "apsp_reduced": (_I32, [_P, _P, _I64, _P, _P]),
     "apsp_reduced_emulated": (_I32, [_P, _I32, _P, _I64, _P]),
+    "ear_owned_tile_rows": (_I32, [_I32, _I32, _I32]),
     "ear_gather_reduced": (_I32, [_P, _P, _I64, _P, _I64, _P, _P]),
     "expand_ears": (_I32, [_P, _P, _I64, _I32, _I32, _P, _I64, _P]),
     "ear_query_pairs": (_I32, [_P, _P, _I64, _I64, _P, _P, _P, _P]),
@@ -219,10 +220,13 @@ def ear_decompose(n: int, src: torch.Tensor, dst: torch.Tensor, w: torch.Tensor,
 
 
 def alloc_D(plan: Plan, comm: Comm | None = None) -> torch.Tensor:
-    """Device buffer for apsp_reduced: full Np x Np (single GPU) or this rank's (Np/P) x Np block."""
-    P = 1 if comm is None else comm.nranks
-    Np = plan.info(P).n_reduced_padded
-    return torch.empty((Np // P, Np), dtype=torch.int32, device="cuda")
+    """Device buffer for apsp_reduced: full Np x Np (single GPU) or this rank's owned tile rows."""
+    if comm is None:
+        Np = plan.info(1).n_reduced_padded
+        return torch.empty((Np, Np), dtype=torch.int32, device="cuda")
+    Np = plan.info(comm.nranks).n_reduced_padded
+    nown = lib().ear_owned_tile_rows(Np, comm.nranks, comm.rank)
+    return torch.empty((max(nown, 1) * TILE, Np), dtype=torch.int32, device="cuda")
 
 
 def apsp_reduced(plan: Plan, D: torch.Tensor, comm: Comm | None = None, stream=None) -> torch.Tensor:

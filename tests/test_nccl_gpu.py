@@ -1,6 +1,7 @@
 """The NCCL path on one GPU: a communicator of ONE rank (torch.distributed nccl process group, NCCL
-unique id from the library) runs the row-block schedule with its real ncclBroadcast per FW round and
-ncclAllGather of D, then the expansion -- bit-exact against the oracle.  (The multi-rank schedule
+unique id from the library) runs the sharded schedule with its real ncclAllReduce(MIN) of the pivot
+row block every FW round and of the final D (and the sharded SSSP Phase II), then the expansion --
+bit-exact against the oracle.  (The multi-rank schedule
 itself is checked on one GPU by test_parity_gpu.py::test_sharded_schedule_emulated.)"""
 import os
 import socket
@@ -22,10 +23,11 @@ dist.init_process_group("nccl", rank=0, world_size=1, device_id=torch.device("cu
 comm = ea.Comm.from_torch_distributed()
 dev = lambda a: torch.as_tensor(np.ascontiguousarray(a, dtype=np.int32)).cuda()
 for g in [gg.config("cfg1"), gg.corner_cases(12, n_target=500)]:
-    out = ea.apsp_full(g.n, dev(g.src), dev(g.dst), dev(g.w), comm=comm)
-    torch.cuda.synchronize()
     ref = oracle.apsp(g.n, g.src, g.dst, g.w)
-    assert np.array_equal(out.cpu().numpy(), ref), "nccl path mismatch"
+    for flags in (0, ea.FLAG_SSSP):
+        out = ea.apsp_full(g.n, dev(g.src), dev(g.dst), dev(g.w), comm=comm, flags=flags)
+        torch.cuda.synchronize()
+        assert np.array_equal(out.cpu().numpy(), ref), f"nccl path mismatch (flags={flags})"
     host = ea.apsp_full_host(g.n, g.src, g.dst, g.w, comm=comm)
     assert np.array_equal(host.numpy(), ref), "nccl host path mismatch"
 comm.destroy()
