@@ -1,3 +1,4 @@
+"""Time expand_ears on a config (device events, 5 repetitions after 2 warm-ups)."""
 import os, sys, time, torch
 sys.path.insert(0,'.')
 import paper_conf_ipps_duttackb17_b200 as ea

@@ -1,3 +1,4 @@
+"""Time Phase II by per-source SSSP on a config; set EAR_SSSP_STATS=1 for round / relaxation counts."""
 import sys, time, torch
 sys.path.insert(0,'.')
 import paper_conf_ipps_duttackb17_b200 as ea
