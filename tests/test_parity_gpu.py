@@ -339,3 +339,12 @@ def test_sssp_cfg4_sampled_rows(pkg):
 def test_sssp_degenerate(pkg, case):
     g = {"n1": graph(1, []), "m0": graph(7, []), "cycle": gg.cycle(9, seed=5), "path": gg.path(40, seed=6)}[case]
     assert_exact(run_full(pkg, g, flags=pkg.FLAG_SSSP), oracle.apsp(g.n, g.src, g.dst, g.w), case)
+
+
+def test_cfg2_random_relabel_full(pkg):
+    """Every entry of the 20k road-like graph with RANDOMLY relabelled vertex ids (no spatial
+    coherence: the expansion's worst case), FW and SSSP Phase II."""
+    g = gg.grid(89, 89, 20000, seed=7, labels="random")
+    ref = oracle.apsp(g.n, g.src, g.dst, g.w)
+    assert_exact(run_full(pkg, g), ref, "cfg2 random labels")
+    assert_exact(run_full(pkg, g, flags=pkg.FLAG_SSSP), ref, "cfg2 random labels sssp")
