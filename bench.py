@@ -5,7 +5,9 @@
 
 One step = one pass of the whole hot path over the workload: apsp_full =
 Reduce(G) chain contraction -> blocked min-plus FW on G^r -> ear expansion of this rank's rows of the
-N x N int32 matrix, graph already resident in HBM.  For N > 1 GPUs (torchrun, one process per GPU)
+N x N int32 matrix, graph already resident in HBM.  By default (--phase2 bcc) Phase II runs the FW on
+the biconnected pieces of G^r and joins them through the articulation points (paper sec. 2.2,
+P:119-131); --phase2 fw runs one FW over all of G^r, --phase2 sssp the per-source SSSP.  For N > 1 GPUs (torchrun, one process per GPU)
 the FW is row-block sharded with a per-round NCCL pivot broadcast and every rank expands its own row
 block; the total work is fixed (strong scaling).  Timing: W untimed warm-up steps, then exactly K
 steps between barrier + synchronize, CUDA events on the launching stream, max over ranks.  D (3.6 GB)
@@ -238,7 +240,13 @@ def run_ours(args, rank, world, local_rank):
     plan.destroy()
     stream = torch.cuda.current_stream(dev)
 
-    flags = ea.FLAG_SSSP if args.phase2 == "sssp" else 0
+    flags = {"fw": 0, "sssp": ea.FLAG_SSSP, "bcc": ea.FLAG_BCC}[args.phase2]
+    bcc = None
+    if args.phase2 == "bcc":
+        pb = ea.ear_decompose(g.n, src, dst, w, flags=flags)
+        bcc = pb.bcc_info()
+        bcc["sum_cubes_over_nr3"] = bcc["sum_cubes"] / float(max(info.n_reduced, 1)) ** 3
+        pb.destroy()
 
     def step():
         ea.apsp_full(g.n, src, dst, w, out=out, row_begin=r0, row_end=r1, flags=flags, comm=comm, stream=stream)
@@ -303,29 +311,33 @@ def run_ours(args, rank, world, local_rank):
                     "note": "label-correcting Bellman-Ford per source; no arithmetic roofline applies"}
     phases = {"decompose": prof["decompose_ms"] / K, "fw": fw_ms / K, "sssp": prof["sssp_ms"] / K, "fw_phase1": prof["fw_phase1_ms"] / K,
               "fw_phase2": prof["fw_phase2_ms"] / K, "fw_phase3": p3_ms / K, "comm": prof["comm_ms"] / K,
-              "expand": ex_ms / K, "same_chain": prof["same_chain_ms"] / K}
+              "expand": ex_ms / K, "same_chain": prof["same_chain_ms"] / K,
+              "bcc_pieces": prof["bcc_pieces_ms"] / K, "compose": prof["compose_ms"] / K}
     fw_minplus = prof["fw_phase2_minplus"] + prof["fw_phase3_minplus"]
     del out
     torch.cuda.empty_cache()
 
-    # Phase II alternative: per-source SSSP on G^r, timed once on the same plan
-    # (bit-identical D; reported beside the north-star FW, not part of the timed steps)
+    # Phase II alternatives (plain FW on all of G^r; SURVEY 8.f NEXT 2 per-source SSSP; NEXT 3 pieces)
+    # (bit-identical D; reported beside the timed Phase II, not part of the timed steps)
     alt = None
-    if args.phase2 == "fw" and world == 1 and not args.no_alt:
-        p2 = ea.ear_decompose(g.n, src, dst, w, flags=ea.FLAG_SSSP)
-        D2 = ea.alloc_D(p2)
-        ea.apsp_reduced(p2, D2)            # warm-up (builds the reduced CSR / ELL once)
-        torch.cuda.synchronize()
-        a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        a0.record(stream)
-        ea.apsp_reduced(p2, D2)
-        a1.record(stream)
-        torch.cuda.synchronize()
-        alt = {"sssp_phase2_ms": a0.elapsed_time(a1), "fw_phase2_ms": fw_ms / K,
-               "note": "Phase II only (D of G^r), same plan; apsp_full --phase2 sssp gives the full step"}
-        del D2
-        p2.destroy()
-        torch.cuda.empty_cache()
+    if world == 1 and not args.no_alt:
+        alt = {"note": "Phase II only (D of G^r), one timed call after a warm-up call; --phase2 X times the full step"}
+        for name, fl in (("fw", 0), ("sssp", ea.FLAG_SSSP), ("bcc", ea.FLAG_BCC)):
+            if name == args.phase2:
+                continue
+            p2 = ea.ear_decompose(g.n, src, dst, w, flags=fl)
+            D2 = ea.alloc_D(p2)
+            ea.apsp_reduced(p2, D2)            # warm-up (builds the reduced CSR / block structure once)
+            torch.cuda.synchronize()
+            a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a0.record(stream)
+            ea.apsp_reduced(p2, D2)
+            a1.record(stream)
+            torch.cuda.synchronize()
+            alt[f"{name}_phase2_ms"] = a0.elapsed_time(a1)
+            del D2
+            p2.destroy()
+            torch.cuda.empty_cache()
 
     # e2e through the host-buffer C-ABI entry point: H2D edges + D2H output rows inside the region
     e2e = None
@@ -367,7 +379,7 @@ def run_ours(args, rank, world, local_rank):
                            "n_chains": info.n_chains, "max_chain_len": info.max_chain_len,
                            "degree2_frac": stats["deg2_frac"], "seed": args.seed, "rows_per_rank": rows,
                            "parallelism": f"row-block x{world}" if world > 1 else "single GPU",
-                           "phase2": args.phase2,
+                           "phase2": args.phase2, "bcc": bcc,
                            "l2": "inputs larger than L2 (D %.1f GB, output %.1f GB per step)" % (
                                4.0 * info.n_reduced_padded ** 2 / 1e9, 4.0 * g.n * g.n / 1e9)},
                 "roofline": roofline, "roofline_expand": roofline_expand,
@@ -389,8 +401,9 @@ def main():
     ap.add_argument("--config", default="cfg4")
     ap.add_argument("--seed", type=int, default=0)
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
-    ap.add_argument("--phase2", choices=["fw", "sssp"], default="fw",
-                    help="Phase II algorithm: blocked FW (north star) or per-source SSSP (SURVEY 8.f NEXT 2)")
+    ap.add_argument("--phase2", choices=["bcc", "fw", "sssp"], default="bcc",
+                    help="Phase II: blocked FW on the biconnected pieces of G^r (paper sec. 2.2, default), "
+                         "blocked FW on all of G^r, or per-source SSSP (SURVEY 8.f NEXT 2)")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--no-cpu-baseline", action="store_true")

@@ -50,8 +50,12 @@ typedef enum {
 enum {
   EAR_FLAG_NONE = 0,
   EAR_FLAG_NO_CONTRACT = 1, /* every vertex is a terminal: direct blocked FW on G (cfg3 baseline) */
-  EAR_FLAG_SSSP = 2         /* Phase II by per-source SSSP on G^r (the paper's own Phase II, P:101;
+  EAR_FLAG_SSSP = 2,        /* Phase II by per-source SSSP on G^r (the paper's own Phase II, P:101;
                                SURVEY 8.f NEXT 2) instead of blocked FW; same D bit for bit */
+  EAR_FLAG_BCC = 4          /* Phase II by biconnected pieces (paper sec. 2.2; SURVEY 8.f
+                               NEXT 3): FW on the largest block of every component and on the pieces
+                               hanging off it, joined through the articulation points; same D
+                               bit for bit.  Exclusive with EAR_FLAG_SSSP. */
 };
 
 typedef struct ear_plan_s *ear_plan_t; /* Reduce(G) result: descriptors + reduced edge list (device) */
@@ -144,6 +148,22 @@ int32_t ear_owned_tile_rows(int32_t n_reduced_padded, int32_t nranks, int32_t ra
 ear_status_t ear_gather_reduced(ear_plan_t plan, const int32_t *d_D_block, int64_t ldd_block,
                                 int32_t *d_D_full, int64_t ldd_full, ear_comm_t comm, void *stream);
 
+/* Block structure of G^r used by EAR_FLAG_BCC (paper sec. 2.2).  Blocks are those of the
+ * simple reduced graph (parallel G^r edges merged).  A "piece" is the largest block of a
+ * connected component (its root piece) or the set of vertices hanging off that block at one
+ * articulation point, with that point (reading C22).  Built on first use: synchronises the plan's
+ * stream.  Errors: EAR_EINVAL (NULL), EAR_ENOMEM, EAR_ECUDA. */
+typedef struct {
+  int32_t n_components;   /* connected components of G^r */
+  int32_t n_blocks;       /* biconnected components with at least one edge */
+  int32_t n_articulation; /* articulation points of G^r */
+  int32_t n_pieces;       /* root pieces + hanging pieces, each solved by its own FW */
+  int32_t largest_piece;  /* vertices of the largest piece */
+  int32_t tree_levels;    /* levels of the BFS spanning forest (latency of the tree sweeps) */
+  double sum_cubes;       /* sum over pieces of size^3 (FW work; N_r^3 without EAR_FLAG_BCC) */
+} ear_bcc_info_t;
+ear_status_t ear_bcc_info(ear_plan_t plan, ear_bcc_info_t *info);
+
 /* ---------------------------------------------------------------- Phase III: UPDATE_DISTANCE
  * Alg. 1 lines 9-11 with the rules of sec. 2.1.3: for rows
  * s in [row_begin, row_end) of S and every column t (caller order):
@@ -213,6 +233,10 @@ typedef struct {
   double sssp_ms;              /* Phase II by per-source SSSP (EAR_FLAG_SSSP) */
   int64_t sssp_launches;
   double sssp_arcs;            /* sources x reduced arcs (one relaxation pass) */
+  double bcc_pieces_ms;        /* EAR_FLAG_BCC: piece matrices init + one-CTA FW of the small pieces
+                                  (large pieces are counted under fw_phase*) */
+  double compose_ms;           /* EAR_FLAG_BCC: S^r rows composed from the pieces */
+  double compose_bytes;        /* 4 * rows * Np written by the compose kernel */
 } ear_profile_t;
 
 void ear_profile_enable(int32_t on);

@@ -91,6 +91,10 @@ ear_status_t ear_decompose(int32_t n, int64_t m, const int32_t *d_src, const int
     set_error("ear_decompose: bad sizes n=%d m=%lld", n, (long long)m);
     return EAR_EINVAL;
   }
+  if ((flags & EAR_FLAG_SSSP) && (flags & EAR_FLAG_BCC)) {
+    set_error("ear_decompose: EAR_FLAG_SSSP and EAR_FLAG_BCC are exclusive");
+    return EAR_EINVAL;
+  }
   ensure_pool();
   ear_plan_s *p = new ear_plan_s;
   cudaGetDevice(&p->device);
@@ -162,6 +166,7 @@ ear_status_t apsp_reduced(ear_plan_t p, int32_t *d_D, int64_t ldd, ear_comm_t co
   cudaStream_t st = (cudaStream_t)stream;
   if (!comm) {
     if (p->flags & EAR_FLAG_SSSP) return sssp_rows(p, d_D, ldd, Np, 0, Np, nullptr, st);
+    if (p->flags & EAR_FLAG_BCC) return bcc_solve(p, nullptr, d_D, ldd, Np, 0, Np, nullptr, st);
     EAR_TRY(fw_init_D(p, d_D, ldd, Np, 0, Np, st));
     return fw_single(d_D, ldd, Np, st);
   }
@@ -173,6 +178,8 @@ ear_status_t apsp_reduced(ear_plan_t p, int32_t *d_D, int64_t ldd, ear_comm_t co
   ear_status_t s = EAR_OK;
   if (p->flags & EAR_FLAG_SSSP) {   // every rank its own rows: no exchange in Phase II
     s = sssp_rows(p, d_D, ldd, Np, 0, nown * TILE, d_rows, st);
+  } else if (p->flags & EAR_FLAG_BCC) {   // largest piece sharded, owned rows composed
+    s = bcc_solve(p, comm, d_D, ldd, Np, 0, nown * TILE, d_rows, st);
   } else {
     std::vector<int32_t> rows(nown);
     if (nown > 0) {
@@ -253,6 +260,10 @@ static ear_status_t solve_rows(ear_plan_s *p, int32_t row_begin, int32_t row_end
     EAR_CUDA_TRY(cudaMallocAsync((void **)&D, sizeof(int32_t) * (size_t)Np * Np, st));
     s = apsp_reduced(p, D, Np, nullptr, st);
     Dfull = D;
+  } else if (p->flags & EAR_FLAG_BCC) {
+    // every rank holds every solved piece after bcc_solve: compose the full matrix directly, no gather
+    EAR_CUDA_TRY(cudaMallocAsync((void **)&Dfull, sizeof(int32_t) * (size_t)Np * Np, st));
+    s = bcc_solve(p, comm, Dfull, Np, Np, 0, Np, nullptr, st);
   } else {
     const int32_t nown = shard_nown(Np / TILE, P, comm->rank);
     EAR_CUDA_TRY(cudaMallocAsync((void **)&Dfull, sizeof(int32_t) * (size_t)Np * Np, st));

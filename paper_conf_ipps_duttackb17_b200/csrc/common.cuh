@@ -40,6 +40,8 @@ struct __align__(16) VDesc {
 
 }  // namespace ear
 
+struct ear_bcc_s;   // bcc.cu: block structure of G^r and the piece layout (EAR_FLAG_BCC)
+
 // Library-owned plan (Reduce(G) result), device arrays unless noted.
 struct ear_plan_s {
   int32_t n = 0;
@@ -70,6 +72,7 @@ struct ear_plan_s {
   void *r_arcs = nullptr;       // packed (col, w) int2 arcs: ELL rows of r_ell_k per vertex, or CSR order
   int32_t r_ell_k = -1;
   int32_t n_rarcs = 0;
+  ear_bcc_s *bcc = nullptr;     // built on first use (EAR_FLAG_BCC, ear_bcc_info)
 };
 
 struct ear_comm_s {
@@ -82,7 +85,7 @@ struct ear_comm_s {
 
 namespace ear {
 // prof.cu
-enum ProfKind { PK_DECOMPOSE, PK_FW_INIT, PK_FW_P1, PK_FW_P2, PK_FW_P3, PK_COMM, PK_EXPAND, PK_SAME_CHAIN, PK_SSSP };
+enum ProfKind { PK_DECOMPOSE, PK_FW_INIT, PK_FW_P1, PK_FW_P2, PK_FW_P3, PK_COMM, PK_EXPAND, PK_SAME_CHAIN, PK_SSSP, PK_BCC, PK_COMPOSE };
 void count_launch(int n = 1);
 int prof_begin(int kind, cudaStream_t s);                // -1 when profiling is off
 void prof_end(int slot, cudaStream_t s, double work);
@@ -111,6 +114,11 @@ ear_status_t shard_rows_device(int32_t nt, int32_t P, int32_t rank, int32_t **d_
 // holds global rows d_tile_rows[b]*128 ..), written consecutively into D
 ear_status_t sssp_rows(ear_plan_s *plan, int32_t *D, int64_t ldd, int32_t Np, int32_t row0, int32_t rows,
                        const int32_t *d_tile_rows, cudaStream_t stream);
+// bcc.cu -- Phase II by biconnected pieces (paper sec. 2.2)
+ear_status_t bcc_prepare(ear_plan_s *plan, int32_t P, cudaStream_t stream);
+ear_status_t bcc_solve(ear_plan_s *plan, ear_comm_s *comm, int32_t *D, int64_t ldd, int32_t Np, int32_t row0,
+                       int32_t rows, const int32_t *d_tile_rows, cudaStream_t stream);
+void bcc_free(ear_bcc_s *b, cudaStream_t stream);
 // expand.cu
 ear_status_t expand(const ear_plan_s *plan, const int32_t *D, int64_t ldd, int32_t row_begin,
                     int32_t row_end, int32_t *out, int64_t ldo, cudaStream_t stream);

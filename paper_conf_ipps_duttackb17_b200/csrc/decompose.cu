@@ -303,6 +303,8 @@ void plan_free(ear_plan_s *p) {
                   p->r_rowptr, p->r_col, p->r_w, p->r_arcs};
   for (void *a : arrs)
     if (a) cudaFreeAsync(a, p->stream);
+  bcc_free(p->bcc, p->stream);
+  p->bcc = nullptr;
 }
 
 template <class T>

@@ -91,6 +91,8 @@ ear_status_t ear_profile_read(ear_profile_t *out) {
       case PK_EXPAND: g_acc.expand_ms += ms; g_acc.expand_launches++; g_acc.expand_bytes += r.work; break;
       case PK_SAME_CHAIN: g_acc.same_chain_ms += ms; break;
       case PK_SSSP: g_acc.sssp_ms += ms; g_acc.sssp_launches++; g_acc.sssp_arcs += r.work; break;
+      case PK_BCC: g_acc.bcc_pieces_ms += ms; break;
+      case PK_COMPOSE: g_acc.compose_ms += ms; g_acc.compose_bytes += r.work; break;
       default: break;
     }
     g_pool.push_back(r.e0);

@@ -27,6 +27,7 @@ TILE = 128
 FLAG_NONE = 0
 FLAG_NO_CONTRACT = 1
 FLAG_SSSP = 2
+FLAG_BCC = 4
 
 _lib = None
 
@@ -50,7 +51,14 @@ class _Profile(ctypes.Structure):
                 ("fw_phase3_minplus", ctypes.c_double), ("comm_ms", ctypes.c_double), ("expand_ms", ctypes.c_double),
                 ("same_chain_ms", ctypes.c_double), ("expand_launches", ctypes.c_int64),
                 ("expand_bytes", ctypes.c_double), ("sssp_ms", ctypes.c_double), ("sssp_launches", ctypes.c_int64),
-                ("sssp_arcs", ctypes.c_double)]
+                ("sssp_arcs", ctypes.c_double), ("bcc_pieces_ms", ctypes.c_double), ("compose_ms", ctypes.c_double),
+                ("compose_bytes", ctypes.c_double)]
+
+
+class _BccInfo(ctypes.Structure):
+    _fields_ = [("n_components", ctypes.c_int32), ("n_blocks", ctypes.c_int32), ("n_articulation", ctypes.c_int32),
+                ("n_pieces", ctypes.c_int32), ("largest_piece", ctypes.c_int32), ("tree_levels", ctypes.c_int32),
+                ("sum_cubes", ctypes.c_double)]
 
 
 # (name, restype, argtypes) for every symbol declared in include/ear_apsp.h
@@ -61,6 +69,7 @@ SIGNATURES = {
     "ear_plan_export": (_I32, [_P, _P, _P, _P, _P, _P, _P, _P]),
     "ear_plan_export_reduced_edges": (_I32, [_P, _P, _P, _P, _P]),
     "ear_plan_destroy": (None, [_P]),
+    "ear_bcc_info": (_I32, [_P, ctypes.POINTER(_BccInfo)]),
     "apsp_reduced": (_I32, [_P, _P, _I64, _P, _P]),
     "apsp_reduced_emulated": (_I32, [_P, _I32, _P, _I64, _P]),
     "ear_owned_tile_rows": (_I32, [_I32, _I32, _I32]),
@@ -182,6 +191,12 @@ class Plan:
         i = _Info()
         _check(lib().ear_plan_info(self.handle, nranks, ctypes.byref(i)), "ear_plan_info")
         return PlanInfo(*[getattr(i, f) for f, _ in _Info._fields_])
+
+    def bcc_info(self) -> dict:
+        """Block structure of G^r used by FLAG_BCC (ear_bcc_info; builds it on first use, synchronises)."""
+        i = _BccInfo()
+        _check(lib().ear_bcc_info(self.handle, ctypes.byref(i)), "ear_bcc_info")
+        return {f: getattr(i, f) for f, _ in _BccInfo._fields_}
 
     def export(self, stream=None) -> dict:
         """Per-vertex descriptors as CUDA int32 tensors (tests)."""

@@ -271,6 +271,96 @@ def corner_cases(seed: int, n_target: int = 60) -> Graph:
     return _finish(n, u, v, None, rng, dict(family="corner_cases", seed=seed), labels="random")
 
 
+def block_tree(seed: int, n_target: int = 200, big: int = 0, chains: bool = True) -> Graph:
+    """Sparse graph made of many biconnected blocks glued at articulation points -- the shape sec. 2.2
+    of the paper is about (real sparse graphs are not 2-connected): cycles, small grids, wheels
+    and theta graphs hung off each other at single vertices, bridges and pendant trees, 1-3 connected
+    components plus isolated vertices.  ``big`` > 0 makes the first block a grid of about ``big``
+    vertices (a dominant block, like the largest BCC of cfg4); ``chains`` subdivides some block
+    edges by degree-two vertices.  Ids are randomly relabelled."""
+    rng = np.random.default_rng(seed)
+    us, vs = [], []
+    n = 0
+
+    def new(k):
+        nonlocal n
+        ids = list(range(n, n + k))
+        n += k
+        return ids
+
+    def edge(a, b):
+        if chains and rng.random() < 0.3:   # subdivide by 1-3 degree-two vertices
+            xs = new(int(rng.integers(1, 4)))
+            seq = [a, *xs, b]
+        else:
+            seq = [a, b]
+        for i in range(len(seq) - 1):
+            us.append(seq[i]); vs.append(seq[i + 1])
+
+    def grid_block(a, gx, gy):
+        ids = [a] + new(gx * gy - 1)
+        for y in range(gy):
+            for x in range(gx):
+                i = y * gx + x
+                if x + 1 < gx:
+                    edge(ids[i], ids[i + 1])
+                if y + 1 < gy:
+                    edge(ids[i], ids[i + gx])
+        return ids
+
+    ncomp = int(rng.integers(1, 4))
+    for c in range(ncomp):
+        goal = n_target * (c + 1) // ncomp
+        if big and c == 0:
+            side = max(2, int(round(big ** 0.5)))
+            pool = grid_block(new(1)[0], side, side)
+        else:
+            pool = new(int(rng.integers(3, 7)))
+            for i in range(len(pool)):
+                edge(pool[i], pool[(i + 1) % len(pool)])
+        while n < goal:
+            a = int(rng.choice(pool))
+            kind = int(rng.integers(0, 6))
+            if kind == 0:                       # cycle through a
+                xs = new(int(rng.integers(2, 7)))
+                seq = [a, *xs, a]
+                for i in range(len(seq) - 1):
+                    edge(seq[i], seq[i + 1])
+                pool += xs
+            elif kind == 1:                     # bridge to a pendant tree
+                xs = new(int(rng.integers(1, 5)))
+                prev = [a]
+                for x in xs:
+                    edge(int(rng.choice(prev)), x)
+                    prev.append(x)
+                pool += xs
+            elif kind == 2:                     # small grid sharing its corner with a
+                pool += grid_block(a, int(rng.integers(2, 4)), int(rng.integers(2, 5)))[1:]
+            elif kind == 3:                     # theta: three internally disjoint a-b paths
+                b = new(1)[0]
+                for _ in range(3):
+                    xs = new(int(rng.integers(0, 3)))
+                    seq = [a, *xs, b]
+                    for i in range(len(seq) - 1):
+                        edge(seq[i], seq[i + 1])
+                    pool += xs
+                pool.append(b)
+            elif kind == 4:                     # wheel with hub a
+                xs = new(int(rng.integers(3, 7)))
+                for i in range(len(xs)):
+                    edge(xs[i], xs[(i + 1) % len(xs)])
+                    edge(a, xs[i])
+                pool += xs
+            else:                               # a chord inside the current component
+                b = int(rng.choice(pool))
+                if b != a and rng.random() < 0.3:
+                    edge(a, b)
+    new(int(rng.integers(0, 4)))               # isolated vertices
+    u = np.array(us, dtype=np.int64)
+    v = np.array(vs, dtype=np.int64)
+    return _finish(n, u, v, None, rng, dict(family="block_tree", seed=seed, big=big), labels="random")
+
+
 # ----------------------------------------------------------------------------------- configs
 # cfg3 torus shapes for the degree-two fraction sweep f (N = 50,000, N_r = 50k (1 - f)).
 CFG3_SHAPES = {0: (200, 250), 20: (200, 200), 40: (150, 200), 60: (100, 200), 80: (100, 100)}
