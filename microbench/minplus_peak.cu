@@ -18,6 +18,7 @@ __device__ __forceinline__ int imad1(int a, int one, int b) {
 // variant 2: half of the accumulators variant 0, half variant 1
 // variant 3: FADD + FMNMX (fp32 on integer values)
 // variant 4: VIADDMNMX.S16x2 (2 ops / instr, 16-bit lanes)
+// variant 5: VIADDMNMX.U16x2 (2 ops / instr, unsigned 16-bit lanes)
 template <int V>
 __global__ void __launch_bounds__(256) mp_kernel(int* out, const int* in, int iters, long long* cyc) {
   int c[NACC];
@@ -48,6 +49,8 @@ __global__ void __launch_bounds__(256) mp_kernel(int* out, const int* in, int it
         c[i] = __float_as_int(fminf(__int_as_float(c[i]), f));
       } else if (V == 4) {
         c[i] = __viaddmin_s16x2(c[(i + 1) % NACC], b0, c[i]);
+      } else if (V == 5) {
+        c[i] = __viaddmin_u16x2(c[(i + 1) % NACC], b0, c[i]);
       }
     }
   }
@@ -86,6 +89,14 @@ int run(const char* name, double ops_per_update, int nsm, int* d_out, int* d_in,
   return 0;
 }
 
+// semantics of the unsigned 16x2 add-min at the top of the range (wrap or saturate?)
+__global__ void u16_semantics(unsigned *out) {
+  const unsigned a[6] = {0x7FFF7FFFu, 0x80008000u, 0xFFFF0001u, 0xC0004000u, 0xFFFEFFFFu, 0x00050003u};
+  const unsigned b[6] = {0x7FFF0001u, 0x80000001u, 0x0001FFFFu, 0x4000C000u, 0x00010001u, 0x00020004u};
+  const unsigned c[6] = {0xFFFFFFFFu, 0xFFFFFFFFu, 0xFFFFFFFFu, 0xFFFFFFFFu, 0xFFFFFFFFu, 0x00060006u};
+  for (int i = 0; i < 6; ++i) out[i] = __viaddmin_u16x2(a[i], b[i], c[i]);
+}
+
 int main() {
   int dev = 0; cudaDeviceProp p; CK(cudaGetDeviceProperties(&p, dev));
   int nsm = p.multiProcessorCount;
@@ -100,6 +111,16 @@ int main() {
   run<2>("mixed_1to1", 1.0, nsm, d_out, d_in, d_cyc);
   run<3>("fadd_fmnmx", 1.0, nsm, d_out, d_in, d_cyc);
   run<4>("viaddmnmx_s16x2", 2.0, nsm, d_out, d_in, d_cyc);
+  run<5>("viaddmnmx_u16x2", 2.0, nsm, d_out, d_in, d_cyc);
+  {
+    unsigned *d_s, h_s[6];
+    CK(cudaMalloc(&d_s, sizeof(h_s)));
+    u16_semantics<<<1, 1>>>(d_s);
+    CK(cudaMemcpy(h_s, d_s, sizeof(h_s), cudaMemcpyDeviceToHost));
+    printf("{\"u16x2_addmin\": [\"%08x\", \"%08x\", \"%08x\", \"%08x\", \"%08x\", \"%08x\"], "
+           "\"inputs\": \"a+b min c for a=7fff7fff+7fff0001, 80008000+80000001, ffff0001+0001ffff, c0004000+4000c000, fffeffff+00010001, 00050003+00020004 (c=00060006)\"}\n",
+           h_s[0], h_s[1], h_s[2], h_s[3], h_s[4], h_s[5]);
+  }
   run<0>("viaddmnmx_again", 1.0, nsm, d_out, d_in, d_cyc);
   return 0;
 }

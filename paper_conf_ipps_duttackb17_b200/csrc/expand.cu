@@ -10,13 +10,24 @@
 //     same chain: S[s, t] = min(S[s, t], |off_s - off_t|)            P:107 (readings C8, C9)
 // then clamped to EAR_INF.
 //
-// k_expand: one CTA per group of RB = 32 consecutive output rows.  The group's distinct chain
-// ends E (<= 64) are split greedily into sub-groups of <= ECAP endpoints; for every 1024-column
-// chunk each thread owns 4 consecutive columns: it builds R[e, its 4 columns] for the sub-group's
-// endpoints in shared memory (2 gathers from the D rows of e each -- the D rows of neighbouring
-// rows' endpoints stay in L1/L2 because caller ids are spatially coherent), then emits every row of
-// the sub-group with two 128-bit shared loads, 3 integer ops per element and one 128-bit streaming
-// store (st.global.cs).  The output is written exactly once: the kernel is HBM-write bound.
+// k_expand: one CTA per group of RB = 32 consecutive output rows; its distinct chain ends E (<= 64)
+// are split greedily into sub-groups of <= ECAP endpoints.  Each of the 8 warps owns a 128-column
+// slice of every 1,024-column chunk and works independently of the others (no CTA barrier in the
+// main loop):
+//   R build   for each end e of the sub-group (4 ends per batch, 32 gathers in flight per lane) and
+//             the slice's columns t -- lane-consecutive, so one gather instruction covers 32
+//             neighbouring columns and few sectors -- R[e, t] = min(D[e,p_t] + cp_t, D[e,q_t] + cq_t)
+//             (2-term rule seen from t) goes to shared memory.  Gathers use one 64-bit row
+//             pointer per end and 32-bit byte offsets per column (2 address instructions each).
+//             When e is itself a terminal row of the sub-group, R[e, .] IS that output row:
+//             it is streamed out right here, never reloaded.
+//   rows      every chain row s of the sub-group: S[s, t] = min(cp_s + R[p_s,t], cq_s + R[q_s,t])
+//             (4-term rule) with two 128-bit shared loads (shared by consecutive rows of one
+//             chain), three integer ops per element and one 128-bit streaming store; row metadata
+//             is one packed int4 per row.
+// The output is written exactly once.  Measured on cfg4 (tools/expand_lab.py, profiles/): the D
+// gathers go to HBM at the first touch of each sector and their latency is what bounds the kernel;
+// with D resident in L2 the same kernel runs at ~90 % of the copy bandwidth.
 // k_same_chain: the P:107 along-chain patch, one warp per row, touching only same-chain entries.
 #include <algorithm>
 
@@ -28,7 +39,8 @@ namespace {
 constexpr int NT = 256;
 constexpr int RB = 32;              // rows per CTA
 constexpr int ECAP = 16;            // endpoints per sub-group (R tile: ECAP x 1024 ints = 64 KB)
-constexpr int CHUNK = NT * 4;       // columns per chunk
+constexpr int CHUNK = 1024;         // columns per chunk (8 warps x 128)
+constexpr int BATCH = 4;            // ends per gather batch
 constexpr int EXP_SMEM = ECAP * CHUNK * 4;
 
 __device__ __forceinline__ void st_cs_v4(int32_t *p, int4 v) {
@@ -42,18 +54,29 @@ __device__ __forceinline__ int32_t out_val(int32_t cp, int32_t rp, int32_t cq, i
   return min(__viaddmin_s32(cq, rq, cp + rp), INF);
 }
 
-template <bool VEC>
-__global__ void __launch_bounds__(NT, 3) k_expand(const int32_t *__restrict__ D, int64_t ldd,
+__device__ __forceinline__ int32_t ldg_off(const int32_t *base, uint32_t byte_off) {
+  return __ldg(reinterpret_cast<const int32_t *>(reinterpret_cast<const char *>(base) + byte_off));
+}
+
+__device__ __forceinline__ int32_t *row_ptr(int32_t *base, int32_t r, uint32_t ld_bytes) {
+  return reinterpret_cast<int32_t *>(reinterpret_cast<char *>(base) + (uint64_t)(uint32_t)r * ld_bytes);
+}
+
+__global__ void __launch_bounds__(NT, 2) k_expand(const int32_t *__restrict__ D, int64_t ldd,
                                                  const VDesc *__restrict__ desc, int32_t n, int32_t row_begin,
                                                  int32_t row_end, int32_t *__restrict__ out, int64_t ldo) {
   extern __shared__ __align__(16) int32_t R[];       // [ECAP][CHUNK]
   __shared__ VDesc rdesc[RB];
   __shared__ int32_t ends[2 * RB];                   // endpoint tids, sub-group by sub-group
+  __shared__ const int32_t *end_ptr[2 * RB];         // their D rows
+  __shared__ int16_t end_row[2 * RB];                // local output row of a terminal end in its sub-group, or -1
   __shared__ int8_t ip[RB], iq[RB];                  // per row: index of p / q in its sub-group
   __shared__ int8_t sg_row0[RB + 1], sg_e0[RB + 1];  // sub-group g: rows [row0[g], row0[g+1]), ends [e0[g], e0[g+1])
+  __shared__ int4 meta[RB];                          // chain rows by sub-group: {cp, cq, ip | iq << 8, local row}
+  __shared__ int8_t sg_m0[RB + 1];
   __shared__ int32_t n_sg;
 
-  const int tid = threadIdx.x;
+  const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
   const int32_t r0 = row_begin + blockIdx.x * RB;
   const int nrows = min(RB, row_end - r0);
   if (tid < nrows) rdesc[tid] = desc[r0 + tid];
@@ -84,86 +107,102 @@ __global__ void __launch_bounds__(NT, 3) k_expand(const int32_t *__restrict__ D,
     ++g;
     sg_row0[g] = (int8_t)nrows; sg_e0[g] = (int8_t)ne;
     n_sg = g;
+    // terminal rows are emitted by the R build of their own end; the rest become chain-row metadata
+    int m = 0;
+    for (int k = 0; k < g; ++k) {
+      sg_m0[k] = (int8_t)m;
+      const int b = sg_e0[k];
+      for (int e = b; e < sg_e0[k + 1]; ++e) end_row[e] = -1;
+      for (int r = sg_row0[k]; r < sg_row0[k + 1]; ++r) {
+        const VDesc d = rdesc[r];
+        if (d.p == d.q && d.cp == 0 && d.cq == 0 && end_row[b + ip[r]] < 0)
+          end_row[b + ip[r]] = (int16_t)r;
+        else
+          meta[m++] = make_int4(d.cp, d.cq, (int)ip[r] | ((int)iq[r] << 8), r);
+      }
+    }
+    sg_m0[g] = (int8_t)m;
   }
   __syncthreads();
+  if (tid < sg_e0[n_sg]) end_ptr[tid] = D + (int64_t)ends[tid] * ldd;
+  __syncthreads();
   const int nsg = n_sg;
-  int32_t *Rt = R + tid * 4;   // this thread's 4 columns in every R row
-
-  for (int32_t c0 = 0; c0 < n; c0 += CHUNK) {
-    const int32_t col = c0 + tid * 4;
-    if (col >= n) break;   // (no barriers below: every thread works on its own columns only)
-    const int ncol = min(4, n - col);
-    int32_t pt[4], cpt[4], qt[4], cqt[4];
+  const bool vec_ok = (ldo & 3) == 0;
+  const uint32_t ldo_b = (uint32_t)(ldo * 4);
+  int32_t *const oblk = out + (int64_t)(r0 - row_begin) * ldo;   // this CTA's first output row
+  int32_t *Rw = R + w * 128;                                       // this warp's slice of every R row
+  for (int32_t c0 = w * 128; c0 < n; c0 += CHUNK) {
+    uint32_t op[4], oq[4];
+    int32_t cpt[4], cqt[4];
 #pragma unroll
     for (int j = 0; j < 4; ++j) {
-      if (j < ncol) {
-        const VDesc d = desc[col + j];
-        pt[j] = d.p; cpt[j] = d.cp; qt[j] = d.q; cqt[j] = d.cq;
-      } else {
-        pt[j] = qt[j] = 0; cpt[j] = cqt[j] = 0;
-      }
+      const int32_t t = c0 + 32 * j + lane;
+      const VDesc d = t < n ? desc[t] : VDesc{0, 0, 0, 0};
+      op[j] = (uint32_t)d.p * 4u; oq[j] = (uint32_t)d.q * 4u; cpt[j] = d.cp; cqt[j] = d.cq;
     }
     for (int g = 0; g < nsg; ++g) {
       const int e0 = sg_e0[g], ne = sg_e0[g + 1] - e0;
-      // R rows for the sub-group's endpoints; 4 endpoints per batch keep 32 independent gathers
-      // in flight per thread (the kernel is otherwise gather-latency bound)
-      int e = 0;
-      for (; e + 4 <= ne; e += 4) {
-        int32_t gp[4][4], gq[4][4];
+      for (int e = 0; e < ne; e += BATCH) {
+        int32_t gp[BATCH][4], gq[BATCH][4];
 #pragma unroll
-        for (int u = 0; u < 4; ++u) {
-          const int32_t *De = D + (int64_t)ends[e0 + e + u] * ldd;
+        for (int u = 0; u < BATCH; ++u) {
+          const int32_t *De = end_ptr[e0 + min(e + u, ne - 1)];   // past the last end: repeat it (cached)
 #pragma unroll
           for (int j = 0; j < 4; ++j) {
-            gp[u][j] = __ldg(De + pt[j]);
-            gq[u][j] = __ldg(De + qt[j]);
+            gp[u][j] = ldg_off(De, op[j]);
+            gq[u][j] = ldg_off(De, oq[j]);
           }
         }
 #pragma unroll
-        for (int u = 0; u < 4; ++u) {
-          int4 v;   // clamped to INF so that cp_s + R below cannot overflow
-          v.x = min(__viaddmin_s32(gq[u][0], cqt[0], gp[u][0] + cpt[0]), INF);
-          v.y = min(__viaddmin_s32(gq[u][1], cqt[1], gp[u][1] + cpt[1]), INF);
-          v.z = min(__viaddmin_s32(gq[u][2], cqt[2], gp[u][2] + cpt[2]), INF);
-          v.w = min(__viaddmin_s32(gq[u][3], cqt[3], gp[u][3] + cpt[3]), INF);
-          *reinterpret_cast<int4 *>(Rt + (e + u) * CHUNK) = v;
-        }
-      }
-      for (; e < ne; ++e) {
-        const int32_t *De = D + (int64_t)ends[e0 + e] * ldd;
-        int4 v;
-        v.x = min(__viaddmin_s32(__ldg(De + qt[0]), cqt[0], __ldg(De + pt[0]) + cpt[0]), INF);
-        v.y = min(__viaddmin_s32(__ldg(De + qt[1]), cqt[1], __ldg(De + pt[1]) + cpt[1]), INF);
-        v.z = min(__viaddmin_s32(__ldg(De + qt[2]), cqt[2], __ldg(De + pt[2]) + cpt[2]), INF);
-        v.w = min(__viaddmin_s32(__ldg(De + qt[3]), cqt[3], __ldg(De + pt[3]) + cpt[3]), INF);
-        *reinterpret_cast<int4 *>(Rt + e * CHUNK) = v;
-      }
-      const int rend = sg_row0[g + 1];
-      int last_p = -1, last_q = -1;
-      int4 a = make_int4(0, 0, 0, 0), b = a;
-      for (int r = sg_row0[g]; r < rend; ++r) {
-        const VDesc s = rdesc[r];
-        const int rp = ip[r], rq = iq[r];
-        if (rp != last_p || rq != last_q) {   // consecutive rows of one chain share their R rows
-          a = *reinterpret_cast<const int4 *>(Rt + rp * CHUNK);
-          b = (rq == rp) ? a : *reinterpret_cast<const int4 *>(Rt + rq * CHUNK);   // terminal rows: one load
-          last_p = rp; last_q = rq;
-        }
-        int4 o;
-        o.x = out_val(s.cp, a.x, s.cq, b.x);
-        o.y = out_val(s.cp, a.y, s.cq, b.y);
-        o.z = out_val(s.cp, a.z, s.cq, b.z);
-        o.w = out_val(s.cp, a.w, s.cq, b.w);
-        int32_t *orow = out + (int64_t)(r0 - row_begin + r) * ldo + col;
-        if (VEC && ncol == 4) {
-          st_cs_v4(orow, o);
-        } else {
-          const int32_t ov[4] = {o.x, o.y, o.z, o.w};
+        for (int u = 0; u < BATCH; ++u) {
+          if (e + u < ne) {
+            int32_t v[4];
 #pragma unroll
-          for (int j = 0; j < 4; ++j)
-            if (j < ncol) orow[j] = ov[j];
+            for (int j = 0; j < 4; ++j) {   // clamped to INF so that cp_s + R below cannot overflow
+              v[j] = min(__viaddmin_s32(gq[u][j], cqt[j], gp[u][j] + cpt[j]), INF);
+              Rw[(e + u) * CHUNK + 32 * j + lane] = v[j];
+            }
+            const int er = end_row[e0 + e + u];
+            if (er >= 0) {   // warp-uniform: a terminal row of this sub-group -- emit it now
+              int32_t *orow = row_ptr(oblk, er, ldo_b);
+#pragma unroll
+              for (int j = 0; j < 4; ++j)
+                if (c0 + 32 * j + lane < n) __stcs(orow + c0 + 32 * j + lane, v[j]);
+            }
+          }
         }
       }
+      __syncwarp();
+      const int32_t col = c0 + lane * 4;
+      const int ncol = max(0, min(4, n - col));
+      const int m1 = sg_m0[g + 1];
+      int32_t *obase = oblk + col;
+      if (ncol == 4 && vec_ok) {
+        int last = -1;
+        int4 a = make_int4(0, 0, 0, 0), b = a;
+        for (int m = sg_m0[g]; m < m1; ++m) {
+          const int4 md = meta[m];
+          if (md.z != last) {   // consecutive rows of one chain share their R rows
+            a = *reinterpret_cast<const int4 *>(Rw + (md.z & 0xFF) * CHUNK + lane * 4);
+            b = *reinterpret_cast<const int4 *>(Rw + (md.z >> 8) * CHUNK + lane * 4);
+            last = md.z;
+          }
+          int4 o;
+          o.x = out_val(md.x, a.x, md.y, b.x);
+          o.y = out_val(md.x, a.y, md.y, b.y);
+          o.z = out_val(md.x, a.z, md.y, b.z);
+          o.w = out_val(md.x, a.w, md.y, b.w);
+          st_cs_v4(row_ptr(obase, md.w, ldo_b), o);
+        }
+      } else if (ncol > 0) {   // ragged tail or unaligned rows
+        for (int m = sg_m0[g]; m < m1; ++m) {
+          const int4 md = meta[m];
+          const int32_t *ra = Rw + (md.z & 0xFF) * CHUNK + lane * 4, *rb = Rw + (md.z >> 8) * CHUNK + lane * 4;
+          int32_t *orow = obase + (int64_t)md.w * ldo;
+          for (int j = 0; j < ncol; ++j) orow[j] = out_val(md.x, ra[j], md.y, rb[j]);
+        }
+      }
+      __syncwarp();
     }
   }
 }
@@ -217,18 +256,13 @@ ear_status_t expand(const ear_plan_s *plan, const int32_t *D, int64_t ldd, int32
   const int32_t rows = row_end - row_begin;
   if (rows <= 0) return EAR_OK;
   if (!g_attr_set) {
-    EAR_CUDA_TRY(cudaFuncSetAttribute(k_expand<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, EXP_SMEM));
-    EAR_CUDA_TRY(cudaFuncSetAttribute(k_expand<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, EXP_SMEM));
+    EAR_CUDA_TRY(cudaFuncSetAttribute(k_expand, cudaFuncAttributeMaxDynamicSharedMemorySize, EXP_SMEM));
     g_attr_set = true;
   }
-  const bool vec = ((uintptr_t)out % 16 == 0) && (ldo % 4 == 0);
   const unsigned grid = (unsigned)ceil_div(rows, RB);
   const double nr = plan->n_reduced;
   int se = prof_begin(PK_EXPAND, st);
-  if (vec)
-    EAR_LAUNCH(k_expand<true>, grid, NT, EXP_SMEM, st)(D, ldd, plan->desc, plan->n, row_begin, row_end, out, ldo);
-  else
-    EAR_LAUNCH(k_expand<false>, grid, NT, EXP_SMEM, st)(D, ldd, plan->desc, plan->n, row_begin, row_end, out, ldo);
+  EAR_LAUNCH(k_expand, grid, NT, EXP_SMEM, st)(D, ldd, plan->desc, plan->n, row_begin, row_end, out, ldo);
   prof_end(se, st, 4.0 * rows * plan->n + 16.0 * plan->n + 4.0 * nr * nr * rows / plan->n);
   if (plan->n_chain_vertices > 0) {
     int ss = prof_begin(PK_SAME_CHAIN, st);
