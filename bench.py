@@ -240,7 +240,7 @@ def run_ours(args, rank, world, local_rank):
     plan.destroy()
     stream = torch.cuda.current_stream(dev)
 
-    flags = {"fw": 0, "sssp": ea.FLAG_SSSP, "bcc": ea.FLAG_BCC}[args.phase2]
+    flags = {"fw": 0, "sssp": ea.FLAG_SSSP, "bcc": ea.FLAG_BCC}[args.phase2] | (ea.FLAG_FW32 if args.fw32 else 0)
     bcc = None
     if args.phase2 == "bcc":
         pb = ea.ear_decompose(g.n, src, dst, w, flags=flags)
@@ -290,8 +290,23 @@ def run_ours(args, rank, world, local_rank):
                 "avg_launch_ms": p3_ms / n_p3, "minplus_per_launch": prof["fw_phase3_minplus"] / n_p3,
                 "peak_basis": f"{SM_COUNT} SMs x {ALU_LANES_PER_SM} VIADDMNMX/clk/SM x {sm_max:.0f} MHz "
                               "(sm_max_mhz of MEASURED_PEAKS.json; issue rate from microbench/minplus_peak.cu)"}
+    lanes = ALU_LANES_PER_SM
+    if prof["fw_phase3_16_minplus"] > 0:
+        # the packed 16-bit FW ran: two min-plus per VIADDMNMX.U16x2 at the same issue
+        # rate (microbench/minplus_peak.cu: 37.15 T/s), so its roofline peak is twice the int32 one
+        lanes = 2 * ALU_LANES_PER_SM
+        p16 = prof["fw_phase3_16_ms"]
+        n16 = max(int(prof["fw_phase3_launches"]), 1)
+        ach = prof["fw_phase3_16_minplus"] / (p16 / 1e3) / 1e12
+        peak_alu = SM_COUNT * lanes * sm_max * 1e6 / 1e12
+        roofline.update({"kernel": "k_fw_tiles16 (FW phase 3, packed u16x2)", "achieved": ach, "peak": peak_alu,
+                         "frac": ach / peak_alu, "traffic": ncu_traffic("k_fw_tiles16", args.config),
+                         "avg_launch_ms": p16 / n16, "minplus_per_launch": prof["fw_phase3_16_minplus"] / n16,
+                         "peak_basis": f"{SM_COUNT} SMs x {lanes} min-plus/clk/SM (64 VIADDMNMX.U16x2, two lanes "
+                                       f"each) x {sm_max:.0f} MHz (sm_max_mhz of MEASURED_PEAKS.json; issue rate "
+                                       "from microbench/minplus_peak.cu)"})
     if clocks.get("sm_mhz"):
-        roofline["frac_at_run_clock"] = ach / (SM_COUNT * ALU_LANES_PER_SM * clocks["sm_mhz"] * 1e6 / 1e12)
+        roofline["frac_at_run_clock"] = ach / (SM_COUNT * lanes * clocks["sm_mhz"] * 1e6 / 1e12)
     hbm = float(peaks.get("hbm_gbs", 6555.2))
     ex_ms = prof["expand_ms"]
     ex_ach = prof["expand_bytes"] / (ex_ms / 1e3) / 1e9 if ex_ms > 0 else 0.0
@@ -300,7 +315,7 @@ def run_ours(args, rank, world, local_rank):
                        "avg_launch_ms": ex_ms / max(prof["expand_launches"], 1),
                        "bytes_per_launch": prof["expand_bytes"] / max(prof["expand_launches"], 1)}
     K = args.steps
-    fw_ms = prof["fw_init_ms"] + prof["fw_phase1_ms"] + prof["fw_phase2_ms"] + prof["fw_phase3_ms"]
+    fw_ms = prof["fw_init_ms"] + prof["fw_phase1_ms"] + prof["fw_phase2_ms"] + prof["fw_phase3_ms"] + prof["fw16_conv_ms"]
     if args.phase2 == "sssp":   # the dominant kernel is the per-source SSSP (latency / L2-atomic bound)
         sssp_ms = prof["sssp_ms"]
         roofline = {"bound": "latency", "kernel": "k_sssp_bf (Phase II by per-source SSSP)",
@@ -312,7 +327,8 @@ def run_ours(args, rank, world, local_rank):
     phases = {"decompose": prof["decompose_ms"] / K, "fw": fw_ms / K, "sssp": prof["sssp_ms"] / K, "fw_phase1": prof["fw_phase1_ms"] / K,
               "fw_phase2": prof["fw_phase2_ms"] / K, "fw_phase3": p3_ms / K, "comm": prof["comm_ms"] / K,
               "expand": ex_ms / K, "same_chain": prof["same_chain_ms"] / K,
-              "bcc_pieces": prof["bcc_pieces_ms"] / K, "compose": prof["compose_ms"] / K}
+              "bcc_pieces": prof["bcc_pieces_ms"] / K, "compose": prof["compose_ms"] / K,
+              "fw16_conv": prof["fw16_conv_ms"] / K}
     fw_minplus = prof["fw_phase2_minplus"] + prof["fw_phase3_minplus"]
     del out
     torch.cuda.empty_cache()
@@ -373,7 +389,9 @@ def run_ours(args, rank, world, local_rank):
     if rank == 0:
         line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": K, "warmup": args.warmup,
                 "ms_per_step": ms_max / K, "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
-                "dtype": "int32", "data": "synthetic (seeded generator, spatially coherent labels)",
+                "dtype": "int32" if prof["fw16_used"] == 0 else "int32 (FW: packed u16x2, exact below 0x7FFF)",
+                "data": "synthetic (seeded generator, spatially coherent labels)",
+                "fw16": {"used": int(prof["fw16_used"]) // K, "fallbacks": int(prof["fw16_fallbacks"]) // K},
                 "config": {"workload": WORKLOADS.get(args.config, args.config), "name": args.config,
                            "n": g.n, "m": g.m, "n_reduced": info.n_reduced, "n_reduced_padded": info.n_reduced_padded,
                            "n_chains": info.n_chains, "max_chain_len": info.max_chain_len,
@@ -404,6 +422,7 @@ def main():
     ap.add_argument("--phase2", choices=["bcc", "fw", "sssp"], default="bcc",
                     help="Phase II: blocked FW on the biconnected pieces of G^r (paper sec. 2.2, default), "
                          "blocked FW on all of G^r, or per-source SSSP (SURVEY 8.f NEXT 2)")
+    ap.add_argument("--fw32", action="store_true", help="int32 FW throughout (EAR_FLAG_FW32)")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--no-cpu-baseline", action="store_true")

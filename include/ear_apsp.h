@@ -52,10 +52,16 @@ enum {
   EAR_FLAG_NO_CONTRACT = 1, /* every vertex is a terminal: direct blocked FW on G (cfg3 baseline) */
   EAR_FLAG_SSSP = 2,        /* Phase II by per-source SSSP on G^r (the paper's own Phase II, P:101;
                                SURVEY 8.f NEXT 2) instead of blocked FW; same D bit for bit */
-  EAR_FLAG_BCC = 4          /* Phase II by biconnected pieces (paper sec. 2.2; SURVEY 8.f
+  EAR_FLAG_BCC = 4,         /* Phase II by biconnected pieces (paper sec. 2.2; SURVEY 8.f
                                NEXT 3): FW on the largest block of every component and on the pieces
                                hanging off it, joined through the articulation points; same D
                                bit for bit.  Exclusive with EAR_FLAG_SSSP. */
+  EAR_FLAG_FW32 = 8         /* single-GPU FW: skip the packed 16-bit attempt and run int32 throughout.
+                               By default the FW first runs on a copy of D capped at 0x7FFF with two
+                               min-plus per VIADDMNMX.U16x2 (exact for every distance < 0x7FFF, see
+                               DESIGN.md sec. 6d) and keeps that result unless a connected pair reached
+                               the cap, in which case it re-runs in int32: D is the same bit for bit
+                               either way.  The range check synchronises the stream once. */
 };
 
 typedef struct ear_plan_s *ear_plan_t; /* Reduce(G) result: descriptors + reduced edge list (device) */
@@ -237,6 +243,11 @@ typedef struct {
                                   (large pieces are counted under fw_phase*) */
   double compose_ms;           /* EAR_FLAG_BCC: S^r rows composed from the pieces */
   double compose_bytes;        /* 4 * rows * Np written by the compose kernel */
+  int64_t fw16_used;           /* FW calls whose packed 16-bit result was kept */
+  int64_t fw16_fallbacks;      /* FW calls where a connected pair reached the 16-bit cap (int32 re-run) */
+  double fw16_conv_ms;         /* 16-bit path: int32 <-> u16 conversions and the range check */
+  double fw_phase3_16_ms;      /* the part of fw_phase3_ms spent in the packed 16-bit tile kernel */
+  double fw_phase3_16_minplus; /* its algorithmic min-plus (two per VIADDMNMX.U16x2) */
 } ear_profile_t;
 
 void ear_profile_enable(int32_t on);

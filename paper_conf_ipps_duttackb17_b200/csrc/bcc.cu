@@ -663,7 +663,6 @@ ear_status_t bcc_prepare(ear_plan_s *p, int32_t P, cudaStream_t st) {
   return EAR_OK;
 }
 
-ear_status_t fw_single(int32_t *D, int64_t ldd, int32_t Np, cudaStream_t st);
 ear_status_t fw_sharded(int32_t *S, int64_t ldd, int32_t Np, ear_comm_s *comm, cudaStream_t st);
 ear_status_t fw_sharded_gather(const int32_t *S, int64_t ldd, int32_t Np, int32_t *Df, int64_t ldf, ear_comm_s *comm,
                                cudaStream_t st);
@@ -717,7 +716,7 @@ ear_status_t bcc_solve(ear_plan_s *p, ear_comm_s *comm, int32_t *D, int64_t ldd,
       if (s == EAR_OK) s = fw_sharded_gather(S, ld, ld, M, ld, comm, st);
       cudaFreeAsync(S, st);
     } else {
-      s = fw_single(M, ld, ld, st);
+      s = fw_single(M, ld, ld, st, nullptr, b->h_psize[id], !(p->flags & EAR_FLAG_FW32));   // a piece is connected
     }
   }
   if (s == EAR_OK) {

@@ -73,6 +73,8 @@ struct ear_plan_s {
   int32_t r_ell_k = -1;
   int32_t n_rarcs = 0;
   ear_bcc_s *bcc = nullptr;     // built on first use (EAR_FLAG_BCC, ear_bcc_info)
+  int32_t *cc = nullptr;        // [cc_np] connected-component labels of G^r (16-bit FW range check)
+  int32_t cc_np = 0;
 };
 
 struct ear_comm_s {
@@ -85,7 +87,9 @@ struct ear_comm_s {
 
 namespace ear {
 // prof.cu
-enum ProfKind { PK_DECOMPOSE, PK_FW_INIT, PK_FW_P1, PK_FW_P2, PK_FW_P3, PK_COMM, PK_EXPAND, PK_SAME_CHAIN, PK_SSSP, PK_BCC, PK_COMPOSE };
+enum ProfKind { PK_DECOMPOSE, PK_FW_INIT, PK_FW_P1, PK_FW_P2, PK_FW_P3, PK_COMM, PK_EXPAND, PK_SAME_CHAIN, PK_SSSP, PK_BCC, PK_COMPOSE,
+                PK_FW_P3_16, PK_FW16_CONV };
+void prof_fw16(bool used);   // one 16-bit FW attempt: used, or fell back to int32
 void count_launch(int n = 1);
 int prof_begin(int kind, cudaStream_t s);                // -1 when profiling is off
 void prof_end(int slot, cudaStream_t s, double work);
@@ -98,7 +102,9 @@ void plan_free(ear_plan_s *plan);
 // fw.cu
 ear_status_t fw_init_D(const ear_plan_s *plan, int32_t *D, int64_t ldd, int32_t Np, int32_t row0,
                        int32_t rows, cudaStream_t stream);
-ear_status_t fw_single(int32_t *D, int64_t ldd, int32_t Np, cudaStream_t stream);
+ear_status_t fw_single(int32_t *D, int64_t ldd, int32_t Np, cudaStream_t stream, const int32_t *lab = nullptr,
+                       int32_t n_real = 0, bool allow16 = false);
+ear_status_t reduced_labels(ear_plan_s *p, int32_t Np, cudaStream_t st, const int32_t **out);
 // row-block sharding: rank r owns the tile rows ti with (ti mod 2P) in {r, 2P-1-r} (zig-zag), stored
 // ascending as 128-row blocks
 ear_status_t fw_sharded(int32_t *S, int64_t ldd, int32_t Np, ear_comm_s *comm, cudaStream_t stream);

@@ -305,6 +305,8 @@ void plan_free(ear_plan_s *p) {
     if (a) cudaFreeAsync(a, p->stream);
   bcc_free(p->bcc, p->stream);
   p->bcc = nullptr;
+  if (p->cc) cudaFreeAsync(p->cc, p->stream);
+  p->cc = nullptr;
 }
 
 template <class T>

@@ -378,11 +378,288 @@ __global__ void k_scatter_upper(const int32_t *S, int64_t ldd, const int32_t *or
     Df[((int64_t)tj * TILE + bx * 32 + yy) * ldf + (int64_t)ti * TILE + by * 32 + lx] = t[lx][yy];
 }
 
+// ------------------------------------------------------------------------------ 16-bit path
+// Packed unsigned 16-bit FW (VIADDMNMX.U16x2: two min-plus per instruction, twice the int32 issue
+// rate; microbench/minplus_peak.cu).  Values are capped at C16 = 0x7FFF: with a, b <= C16 the
+// 16-bit sum a + b <= 0xFFFE never wraps, and FW over capped values yields exactly min(d, C16) for
+// every pair (min(min(a,C)+min(b,C), C) = min(a+b, C) for a, b >= 0, so the cap commutes with every
+// relaxation).  Hence every entry < C16 is the exact distance; an entry == C16 is exact (unreachable)
+// iff its two vertices lie in different components -- checked afterwards, with a fall back to the
+// int32 FW on the untouched int32 D when some connected pair reached the cap.
+constexpr uint32_t C16 = 0x7FFF;
+
+__global__ void k_to16(const int32_t *__restrict__ D, int64_t ldd, uint16_t *__restrict__ D16, int32_t Np) {
+  const int64_t total = (int64_t)Np * (Np / 4);
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
+    const int32_t r = (int32_t)(i / (Np / 4)), c4 = (int32_t)(i % (Np / 4)) * 4;
+    const int4 v = *reinterpret_cast<const int4 *>(D + (int64_t)r * ldd + c4);
+    const uint32_t lo = (uint32_t)min(v.x, (int32_t)C16) | ((uint32_t)min(v.y, (int32_t)C16) << 16);
+    const uint32_t hi = (uint32_t)min(v.z, (int32_t)C16) | ((uint32_t)min(v.w, (int32_t)C16) << 16);
+    *reinterpret_cast<uint2 *>(D16 + (int64_t)r * Np + c4) = make_uint2(lo, hi);
+  }
+}
+
+// capped entries of connected pairs (lab[i] == lab[j]; only vertices < n_real, labels may be null:
+// then [0, n_real) is one component) -> *bad
+__global__ void k_check16(const uint16_t *__restrict__ D16, int32_t Np, const int32_t *__restrict__ lab, int32_t n_real,
+                          int32_t *bad) {
+  const int64_t total = (int64_t)Np * (Np / 8);
+  int found = 0;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
+    const int32_t r = (int32_t)(i / (Np / 8)), c8 = (int32_t)(i % (Np / 8)) * 8;
+    if (r >= n_real || c8 >= n_real) continue;
+    const uint4 v = *reinterpret_cast<const uint4 *>(D16 + (int64_t)r * Np + c8);
+    const uint32_t w[4] = {v.x, v.y, v.z, v.w};
+#pragma unroll
+    for (int k = 0; k < 8; ++k) {
+      const uint32_t x = (w[k >> 1] >> ((k & 1) * 16)) & 0xFFFFu;
+      const int32_t c = c8 + k;
+      if (x == C16 && c < n_real && (!lab || lab[r] == lab[c])) found = 1;
+    }
+  }
+  if (__syncthreads_or(found) && threadIdx.x == 0) atomicOr(bad, 1);
+}
+
+__global__ void k_from16(const uint16_t *__restrict__ D16, int32_t Np, int32_t *__restrict__ D, int64_t ldd) {
+  const int64_t total = (int64_t)Np * (Np / 4);
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
+    const int32_t r = (int32_t)(i / (Np / 4)), c4 = (int32_t)(i % (Np / 4)) * 4;
+    const uint2 v = *reinterpret_cast<const uint2 *>(D16 + (int64_t)r * Np + c4);
+    auto f = [](uint32_t x) { return x == C16 ? INF : (int32_t)x; };
+    *reinterpret_cast<int4 *>(D + (int64_t)r * ldd + c4) =
+        make_int4(f(v.x & 0xFFFFu), f(v.x >> 16), f(v.y & 0xFFFFu), f(v.y >> 16));
+  }
+}
+
+// Pd[r][c] = P16[r][c] duplicated into both halves (the B operand of the packed product)
+__global__ void k_dup16(const uint16_t *__restrict__ P16, int32_t Np, uint32_t *__restrict__ Pd) {
+  const int64_t total = (int64_t)TILE * (Np / 4);
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
+    const uint2 v = reinterpret_cast<const uint2 *>(P16)[i];
+    reinterpret_cast<uint4 *>(Pd)[i] = make_uint4((v.x & 0xFFFFu) * 0x10001u, (v.x >> 16) * 0x10001u,
+                                                  (v.y & 0xFFFFu) * 0x10001u, (v.y >> 16) * 0x10001u);
+  }
+}
+
+// closure of the 16-bit pivot tile (ld Np), computed in int32 registers (values <= C16, so sums fit)
+__global__ void __launch_bounds__(NT, 1) k_fw_phase1_16(uint16_t *T, int64_t ldt) {
+  __shared__ __align__(16) int32_t rowbuf[2][TILE];
+  const int tx = threadIdx.x & 15, ty = threadIdx.x >> 4;
+  int32_t c[8][8];
+#pragma unroll
+  for (int r = 0; r < 8; ++r) {
+    const int i = (r < 4 ? 0 : 64) + ty * 4 + (r & 3);
+    const uint2 lo = *reinterpret_cast<const uint2 *>(T + (int64_t)i * ldt + tx * 4);
+    const uint2 hi = *reinterpret_cast<const uint2 *>(T + (int64_t)i * ldt + 64 + tx * 4);
+    c[r][0] = lo.x & 0xFFFF; c[r][1] = lo.x >> 16; c[r][2] = lo.y & 0xFFFF; c[r][3] = lo.y >> 16;
+    c[r][4] = hi.x & 0xFFFF; c[r][5] = hi.x >> 16; c[r][6] = hi.y & 0xFFFF; c[r][7] = hi.y >> 16;
+  }
+  if (ty == 0) {
+    *reinterpret_cast<int4 *>(&rowbuf[0][tx * 4]) = make_int4(c[0][0], c[0][1], c[0][2], c[0][3]);
+    *reinterpret_cast<int4 *>(&rowbuf[0][64 + tx * 4]) = make_int4(c[0][4], c[0][5], c[0][6], c[0][7]);
+  }
+  __syncthreads();
+  for (int kk = 0; kk < TILE; ++kk) {
+    const int32_t *rb = rowbuf[kk & 1];
+    const int4 alo = *reinterpret_cast<const int4 *>(rb + ty * 4);
+    const int4 ahi = *reinterpret_cast<const int4 *>(rb + 64 + ty * 4);
+    const int4 blo = *reinterpret_cast<const int4 *>(rb + tx * 4);
+    const int4 bhi = *reinterpret_cast<const int4 *>(rb + 64 + tx * 4);
+    const int32_t a[8] = {alo.x, alo.y, alo.z, alo.w, ahi.x, ahi.y, ahi.z, ahi.w};
+    const int32_t b[8] = {blo.x, blo.y, blo.z, blo.w, bhi.x, bhi.y, bhi.z, bhi.w};
+#pragma unroll
+    for (int r = 0; r < 8; ++r)
+#pragma unroll
+      for (int q = 0; q < 8; ++q) c[r][q] = mp(a[r], b[q], c[r][q]);
+    const int nk = kk + 1;
+    if (nk < TILE && ty == ((nk & 63) >> 2)) {
+      const int rr = (nk & 3) + (nk >= 64 ? 4 : 0);
+      int32_t *wb = rowbuf[nk & 1];
+#pragma unroll
+      for (int r = 0; r < 8; ++r) {
+        if (r == rr) {
+          *reinterpret_cast<int4 *>(wb + tx * 4) = make_int4(c[r][0], c[r][1], c[r][2], c[r][3]);
+          *reinterpret_cast<int4 *>(wb + 64 + tx * 4) = make_int4(c[r][4], c[r][5], c[r][6], c[r][7]);
+        }
+      }
+    }
+    __syncthreads();
+  }
+#pragma unroll
+  for (int r = 0; r < 8; ++r) {
+    const int i = (r < 4 ? 0 : 64) + ty * 4 + (r & 3);
+    auto pk = [&](int q) { return (uint32_t)min(c[r][q], (int32_t)C16) | ((uint32_t)min(c[r][q + 1], (int32_t)C16) << 16); };
+    *reinterpret_cast<uint2 *>(T + (int64_t)i * ldt + tx * 4) = make_uint2(pk(0), pk(2));
+    *reinterpret_cast<uint2 *>(T + (int64_t)i * ldt + 64 + tx * 4) = make_uint2(pk(4), pk(6));
+  }
+}
+
+// Phases 2 and 3, packed: the same persistent TMA-ring structure as k_fw_tiles.  A^T chunks are 16-bit
+// rows of the pivot row block (tmA: KC x 128 u16), B chunks rows of its duplicated copy Pd (tmB: KC x
+// 128 u32).  Thread (ty, tx) owns rows {ty*4 .. +3, 64 + ty*4 .. +3} as 4 row PAIRS and columns
+// {tx*4 .. +3, 64 + tx*4 .. +3}: c[r2][q] = (C[i][j], C[i+1][j]) packed, so one VIADDMNMX.U16x2
+// c = min(c, a_pair + b_dup) does two min-plus.
+struct TileJob16 {
+  uint16_t *C;       // matrix holding the C tiles, leading dimension ldc (u16 elements)
+  int64_t ldc;
+  int32_t a_row0;    // row of the pivot row block inside tmA
+  int32_t k, nt;
+  int32_t mode;      // MODE_PIVOT_ROW or MODE_UPPER
+  int32_t mirror;
+  int64_t ntiles;
+};
+
+template <int KC, int STAGES, int MINB, int UNR>
+struct Fw16Cfg {
+  static constexpr int NCHUNK = TILE / KC;
+  static constexpr int A_CHUNK = KC * TILE;   // u16 elements
+  static constexpr int B_CHUNK = KC * TILE;   // u32 elements
+  static constexpr int SMEM = STAGES * (A_CHUNK * 2 + B_CHUNK * 4) + 2 * STAGES * 8;
+  static constexpr int kKC = KC, kSTAGES = STAGES, kMINB = MINB, kUNR = UNR;
+};
+
+__device__ __forceinline__ void decode16(const TileJob16 &J, int64_t idx, int &ti, int &tj) {
+  TileJob T{};
+  T.k = J.k; T.nt = J.nt; T.mode = J.mode; T.ti0 = 0;
+  int lr;
+  decode_tile(T, idx, ti, tj, lr);
+}
+
+template <class CF>
+__global__ void __launch_bounds__(NT, CF::kMINB)
+    k_fw_tiles16(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB, const TileJob16 J) {
+  constexpr int KC = CF::kKC, NCHUNK = CF::NCHUNK, STAGES = CF::kSTAGES;
+  extern __shared__ __align__(128) uint8_t smem16[];
+  uint16_t *sA = reinterpret_cast<uint16_t *>(smem16);                        // [STAGES][KC][TILE] u16
+  uint32_t *sB = reinterpret_cast<uint32_t *>(sA + STAGES * CF::A_CHUNK);     // [STAGES][KC][TILE] u32
+  uint64_t *full = reinterpret_cast<uint64_t *>(sB + STAGES * CF::B_CHUNK);
+  uint64_t *empty = full + STAGES;
+  const int tid = threadIdx.x, lane = tid & 31;
+  const int tx = tid & 15, ty = tid >> 4;
+
+  const int my_tiles = J.ntiles > (int64_t)blockIdx.x ? (int)((J.ntiles - 1 - blockIdx.x) / gridDim.x + 1) : 0;
+  const int total_chunks = my_tiles * NCHUNK;
+  int issued = 0;
+  auto tile_of = [&](int it, int &ti, int &tj) { decode16(J, blockIdx.x + (int64_t)it * gridDim.x, ti, tj); };
+  auto produce = [&](int upto) {
+    while (issued < upto) {
+      const int st = issued % STAGES;
+      if (issued >= STAGES) mbar_wait(&empty[st], (uint32_t)((issued / STAGES - 1) & 1));
+      int pti, ptj;
+      tile_of(issued / NCHUNK, pti, ptj);
+      const int kc = issued % NCHUNK;
+      mbar_arrive_tx(&full[st], CF::A_CHUNK * 2 + CF::B_CHUNK * 4);
+      tma_load_2d(sA + st * CF::A_CHUNK, &tmA, pti * TILE, J.a_row0 + kc * KC, &full[st]);
+      tma_load_2d(sB + st * CF::B_CHUNK, &tmB, ptj * TILE, kc * KC, &full[st]);
+      ++issued;
+    }
+  };
+  if (tid == 0) {
+    for (int s = 0; s < STAGES; ++s) {
+      mbar_init(&full[s], 1);
+      mbar_init(&empty[s], NT / 32);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
+    asm volatile("prefetch.tensormap [%0];\n" ::"l"(reinterpret_cast<uint64_t>(&tmA)) : "memory");
+    asm volatile("prefetch.tensormap [%0];\n" ::"l"(reinterpret_cast<uint64_t>(&tmB)) : "memory");
+  }
+  __syncthreads();
+  if (tid == 0 && my_tiles > 0) produce(total_chunks < STAGES ? total_chunks : STAGES);
+
+  int g = 0;
+  for (int it = 0; it < my_tiles; ++it) {
+    int ti, tj;
+    tile_of(it, ti, tj);
+    uint32_t c[4][8];
+    uint16_t *Ct = J.C + (int64_t)ti * TILE * J.ldc + (int64_t)tj * TILE;
+#pragma unroll
+    for (int r2 = 0; r2 < 4; ++r2) {
+      const int i = (r2 < 2 ? 0 : 64) + ty * 4 + (r2 & 1) * 2;
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        const uint2 v = *reinterpret_cast<const uint2 *>(Ct + (int64_t)i * J.ldc + h * 64 + tx * 4);
+        const uint2 w = *reinterpret_cast<const uint2 *>(Ct + (int64_t)(i + 1) * J.ldc + h * 64 + tx * 4);
+        c[r2][h * 4 + 0] = __byte_perm(v.x, w.x, 0x5410);
+        c[r2][h * 4 + 1] = __byte_perm(v.x, w.x, 0x7632);
+        c[r2][h * 4 + 2] = __byte_perm(v.y, w.y, 0x5410);
+        c[r2][h * 4 + 3] = __byte_perm(v.y, w.y, 0x7632);
+      }
+    }
+#pragma unroll 1
+    for (int kc = 0; kc < NCHUNK; ++kc, ++g) {
+      if (tid == 0) produce(g + STAGES < total_chunks ? g + STAGES : total_chunks);
+      const int st = g % STAGES;
+      mbar_wait(&full[st], (uint32_t)((g / STAGES) & 1));
+      const uint16_t *a_s = sA + st * CF::A_CHUNK;
+      const uint32_t *b_s = sB + st * CF::B_CHUNK;
+#pragma unroll CF::kUNR
+      for (int kk = 0; kk < KC; ++kk) {
+        const uint2 alo = *reinterpret_cast<const uint2 *>(a_s + kk * TILE + ty * 4);
+        const uint2 ahi = *reinterpret_cast<const uint2 *>(a_s + kk * TILE + 64 + ty * 4);
+        const uint4 blo = *reinterpret_cast<const uint4 *>(b_s + kk * TILE + tx * 4);
+        const uint4 bhi = *reinterpret_cast<const uint4 *>(b_s + kk * TILE + 64 + tx * 4);
+        const uint32_t a[4] = {alo.x, alo.y, ahi.x, ahi.y};
+        const uint32_t b[8] = {blo.x, blo.y, blo.z, blo.w, bhi.x, bhi.y, bhi.z, bhi.w};
+#pragma unroll
+        for (int r2 = 0; r2 < 4; ++r2)
+#pragma unroll
+          for (int q = 0; q < 8; ++q) c[r2][q] = __viaddmin_u16x2(a[r2], b[q], c[r2][q]);
+      }
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&empty[st]);
+    }
+#pragma unroll
+    for (int r2 = 0; r2 < 4; ++r2) {
+      const int i = (r2 < 2 ? 0 : 64) + ty * 4 + (r2 & 1) * 2;
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        const uint32_t *cc = &c[r2][h * 4];
+        *reinterpret_cast<uint2 *>(Ct + (int64_t)i * J.ldc + h * 64 + tx * 4) =
+            make_uint2(__byte_perm(cc[0], cc[1], 0x5410), __byte_perm(cc[2], cc[3], 0x5410));
+        *reinterpret_cast<uint2 *>(Ct + (int64_t)(i + 1) * J.ldc + h * 64 + tx * 4) =
+            make_uint2(__byte_perm(cc[0], cc[1], 0x7632), __byte_perm(cc[2], cc[3], 0x7632));
+      }
+    }
+    if (J.mirror && ti != tj) {
+      uint16_t *Mt = J.C + (int64_t)tj * TILE * J.ldc + (int64_t)ti * TILE;
+#pragma unroll
+      for (int q = 0; q < 8; ++q) {
+        const int j = (q < 4 ? 0 : 64) + tx * 4 + (q & 3);
+        *reinterpret_cast<uint2 *>(Mt + (int64_t)j * J.ldc + ty * 4) = make_uint2(c[0][q], c[1][q]);
+        *reinterpret_cast<uint2 *>(Mt + (int64_t)j * J.ldc + 64 + ty * 4) = make_uint2(c[2][q], c[3][q]);
+      }
+    }
+  }
+}
+
+// connected-component labels (min vertex id) of the reduced graph by hooking + pointer jumping
+__global__ void k_cc_init(int32_t *lab, int32_t n) {
+  for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x)
+    lab[v] = (int32_t)v;
+}
+__global__ void k_cc_hook16(const int32_t *u, const int32_t *v, int64_t E, int32_t *lab, int32_t *changed) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < E; i += (int64_t)gridDim.x * blockDim.x) {
+    const int32_t a = lab[u[i]], b = lab[v[i]];
+    if (a != b) {
+      const int32_t hi = max(a, b), lo = min(a, b);
+      if (atomicMin(&lab[hi], lo) > lo) *changed = 1;
+    }
+  }
+}
+__global__ void k_cc_jump16(int32_t *lab, int32_t n) {
+  for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
+    int32_t l = lab[v];
+    while (lab[l] != l) l = lab[l];
+    lab[v] = l;
+  }
+}
+
 int g_num_sms = 0;
 PFN_cuTensorMapEncodeTiled_v12000 g_encode = nullptr;
 
-// 2-D int32 tensor map over rows x cols (leading dimension ld elements) with a box_rows x 128 box
-ear_status_t make_map(CUtensorMap *map, const int32_t *base, int64_t rows, int64_t cols, int64_t ld, int box_rows) {
+// 2-D tensor map over rows x cols (leading dimension ld elements of elem bytes) with a box_rows x 128 box
+ear_status_t make_map_t(CUtensorMap *map, CUtensorMapDataType dt, int elem, const void *base, int64_t rows,
+                        int64_t cols, int64_t ld, int box_rows) {
   if (!g_encode) {
     cudaDriverEntryPointQueryResult q;
     void *fn = nullptr;
@@ -394,18 +671,21 @@ ear_status_t make_map(CUtensorMap *map, const int32_t *base, int64_t rows, int64
     g_encode = (PFN_cuTensorMapEncodeTiled_v12000)fn;
   }
   cuuint64_t dims[2] = {(cuuint64_t)cols, (cuuint64_t)rows};
-  cuuint64_t strides[1] = {(cuuint64_t)ld * sizeof(int32_t)};
+  cuuint64_t strides[1] = {(cuuint64_t)ld * elem};
   cuuint32_t box[2] = {(cuuint32_t)TILE, (cuuint32_t)box_rows};
   cuuint32_t estr[2] = {1, 1};
-  CUresult r = g_encode(map, CU_TENSOR_MAP_DATA_TYPE_INT32, 2, (void *)base, dims, strides, box, estr,
-                        CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
-                        CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  CUresult r = g_encode(map, dt, 2, const_cast<void *>(base), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                        CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   if (r != CUDA_SUCCESS) {
     set_error("cuTensorMapEncodeTiled failed (%d) rows=%lld cols=%lld ld=%lld", (int)r, (long long)rows,
               (long long)cols, (long long)ld);
     return EAR_ECUDA;
   }
   return EAR_OK;
+}
+
+ear_status_t make_map(CUtensorMap *map, const int32_t *base, int64_t rows, int64_t cols, int64_t ld, int box_rows) {
+  return make_map_t(map, CU_TENSOR_MAP_DATA_TYPE_INT32, 4, base, rows, cols, ld, box_rows);
 }
 
 // The tile kernel's configuration, chosen by measurement on the B200 (cfg4, phase-3 share of the
@@ -441,6 +721,104 @@ ear_status_t launch_tiles(const CUtensorMap &map, TileJob J, int64_t nblocks, cu
   return launch_cfg<FwTile>(map, J, nblocks, st);
 }
 
+
+// Packed 16-bit tile kernel configuration: 64-deep k-chunks, 2-stage ring (96 KB), kk unrolled 16x.
+using Fw16Tile = Fw16Cfg<64, 2, 1, 16>;
+
+template <class CF>
+ear_status_t launch16(const CUtensorMap &mA, const CUtensorMap &mB, TileJob16 J, int64_t nblocks, cudaStream_t st) {
+  if (nblocks <= 0) return EAR_OK;
+  static bool attr = false;
+  if (!attr) {
+    EAR_CUDA_TRY(cudaFuncSetAttribute(k_fw_tiles16<CF>, cudaFuncAttributeMaxDynamicSharedMemorySize, CF::SMEM));
+    attr = true;
+  }
+  int per_sm = 0;
+  EAR_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_fw_tiles16<CF>, NT, CF::SMEM));
+  if (per_sm < 1) per_sm = 1;
+  J.ntiles = nblocks;
+  const int64_t grid = std::min<int64_t>(nblocks, (int64_t)g_num_sms * per_sm);
+  EAR_LAUNCH(k_fw_tiles16<CF>, (unsigned)grid, NT, CF::SMEM, st)(mA, mB, J);
+  return EAR_OK;
+}
+
+int grid_for(int64_t n) { return (int)std::max<int64_t>(1, std::min<int64_t>(ceil_div(n, 256), 148 * 16)); }
+
+// The packed 16-bit FW on a copy of D (see C16 above).  *done = false (D untouched) when a connected
+// pair reached the cap; the caller then runs the int32 FW.  Synchronises the stream once (the check).
+ear_status_t fw_single16(int32_t *D, int64_t ldd, int32_t Np, const int32_t *lab, int32_t n_real, bool *done,
+                         cudaStream_t st) {
+  *done = false;
+  if (!g_num_sms) {
+    int dev = 0;
+    EAR_CUDA_TRY(cudaGetDevice(&dev));
+    EAR_CUDA_TRY(cudaDeviceGetAttribute(&g_num_sms, cudaDevAttrMultiProcessorCount, dev));
+  }
+  const int nt = Np / TILE;
+  const double tile_ops = (double)TILE * TILE * TILE;
+  uint16_t *D16 = nullptr;
+  uint32_t *Pd = nullptr;
+  int32_t *bad = nullptr;
+  if (cudaMallocAsync((void **)&D16, sizeof(uint16_t) * (size_t)Np * Np, st) != cudaSuccess ||
+      cudaMallocAsync((void **)&Pd, sizeof(uint32_t) * (size_t)TILE * Np, st) != cudaSuccess ||
+      cudaMallocAsync((void **)&bad, sizeof(int32_t), st) != cudaSuccess) {
+    cudaGetLastError();
+    if (D16) cudaFreeAsync(D16, st);
+    if (Pd) cudaFreeAsync(Pd, st);
+    return EAR_OK;   // no room for the 16-bit copy: the int32 path runs
+  }
+  ear_status_t s = EAR_OK;
+  CUtensorMap mA, mB;
+  s = make_map_t(&mA, CU_TENSOR_MAP_DATA_TYPE_UINT16, 2, D16, Np, Np, Np, Fw16Tile::kKC);
+  if (s == EAR_OK) s = make_map_t(&mB, CU_TENSOR_MAP_DATA_TYPE_UINT32, 4, Pd, TILE, Np, Np, Fw16Tile::kKC);
+  const int64_t ndup = (int64_t)TILE * (Np / 4);
+  if (s == EAR_OK) {
+    int sc = prof_begin(PK_FW16_CONV, st);
+    EAR_LAUNCH(k_to16, grid_for((int64_t)Np * (Np / 4)), 256, 0, st)(D, ldd, D16, Np);
+    prof_end(sc, st, 0);
+  }
+  for (int k = 0; k < nt && s == EAR_OK; ++k) {
+    uint16_t *P16 = D16 + (int64_t)k * TILE * Np;
+    int s1 = prof_begin(PK_FW_P1, st);
+    EAR_LAUNCH(k_fw_phase1_16, 1, NT, 0, st)(P16 + (int64_t)k * TILE, Np);
+    prof_end(s1, st, tile_ops);
+    int s2 = prof_begin(PK_FW_P2, st);
+    EAR_LAUNCH(k_dup16, grid_for(ndup), 256, 0, st)(P16, Np, Pd);
+    TileJob16 J{D16, Np, k * TILE, k, nt, MODE_PIVOT_ROW, 1, 0};
+    s = launch16<Fw16Tile>(mA, mB, J, nt - 1, st);
+    if (s == EAR_OK) EAR_LAUNCH(k_dup16, grid_for(ndup), 256, 0, st)(P16, Np, Pd);
+    prof_end(s2, st, (nt - 1) * tile_ops);
+    if (s != EAR_OK) break;
+    J.mode = MODE_UPPER;
+    const int64_t nup = (int64_t)(nt - 1) * nt / 2;
+    int s3 = prof_begin(PK_FW_P3_16, st);
+    s = launch16<Fw16Tile>(mA, mB, J, nup, st);
+    prof_end(s3, st, nup * tile_ops);
+  }
+  int32_t h_bad = 1;
+  if (s == EAR_OK) {
+    int sc = prof_begin(PK_FW16_CONV, st);
+    cudaMemsetAsync(bad, 0, sizeof(int32_t), st);
+    EAR_LAUNCH(k_check16, grid_for((int64_t)Np * (Np / 8)), 256, 0, st)(D16, Np, lab, n_real, bad);
+    prof_end(sc, st, 0);
+    cudaError_t e = cudaMemcpyAsync(&h_bad, bad, sizeof(int32_t), cudaMemcpyDeviceToHost, st);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+    if (e != cudaSuccess) { set_error("fw_single16: %s", cudaGetErrorString(e)); s = EAR_ECUDA; }
+  }
+  if (s == EAR_OK && h_bad == 0) {
+    int sc = prof_begin(PK_FW16_CONV, st);
+    EAR_LAUNCH(k_from16, grid_for((int64_t)Np * (Np / 4)), 256, 0, st)(D16, Np, D, ldd);
+    prof_end(sc, st, 0);
+    *done = true;
+  }
+  cudaFreeAsync(D16, st);
+  cudaFreeAsync(Pd, st);
+  cudaFreeAsync(bad, st);
+  if (s != EAR_OK) return s;
+  EAR_CUDA_TRY(cudaGetLastError());
+  return EAR_OK;
+}
+
 }  // namespace
 
 ear_status_t fw_init_D(const ear_plan_s *plan, int32_t *D, int64_t ldd, int32_t Np, int32_t row0, int32_t rows,
@@ -458,8 +836,17 @@ ear_status_t fw_init_D(const ear_plan_s *plan, int32_t *D, int64_t ldd, int32_t 
   return EAR_OK;
 }
 
-// Single GPU: full symmetric D (Np x Np).
-ear_status_t fw_single(int32_t *D, int64_t ldd, int32_t Np, cudaStream_t st) {
+// Single GPU: full symmetric D (Np x Np).  With allow16 the packed 16-bit FW runs first on a copy and
+// its result is kept when no connected pair (labels lab over [0, n_real), or one component when lab is
+// NULL) reached the 16-bit cap; otherwise, or without allow16, the int32 FW below runs.
+ear_status_t fw_single(int32_t *D, int64_t ldd, int32_t Np, cudaStream_t st, const int32_t *lab, int32_t n_real,
+                       bool allow16) {
+  if (allow16 && Np >= 2 * TILE) {
+    bool done = false;
+    EAR_TRY(fw_single16(D, ldd, Np, lab, n_real, &done, st));
+    prof_fw16(done);
+    if (done) return EAR_OK;
+  }
   const int nt = Np / TILE;
   const double tile_ops = (double)TILE * TILE * TILE;
   CUtensorMap map;
@@ -695,6 +1082,35 @@ ear_status_t fw_sharded_emulated(const ear_plan_s *plan, int32_t *D, int64_t ldd
   }
   if (status != EAR_OK) return status;
   EAR_CUDA_TRY(cudaGetLastError());
+  return EAR_OK;
+}
+
+// connected-component labels of G^r (cached in the plan; padding vertices are their own component)
+ear_status_t reduced_labels(ear_plan_s *p, int32_t Np, cudaStream_t st, const int32_t **out) {
+  if (!p->cc || p->cc_np != Np) {
+    if (p->cc) cudaFreeAsync(p->cc, st);
+    p->cc = nullptr;
+    int32_t *changed = nullptr;
+    EAR_CUDA_TRY(cudaMallocAsync((void **)&p->cc, sizeof(int32_t) * (size_t)Np, st));
+    EAR_CUDA_TRY(cudaMallocAsync((void **)&changed, sizeof(int32_t), st));
+    p->cc_np = Np;
+    EAR_LAUNCH(k_cc_init, grid_for(Np), 256, 0, st)(p->cc, Np);
+    ear_status_t s = EAR_OK;
+    for (int it = 0; it < 64 && s == EAR_OK; ++it) {
+      int32_t h = 0;
+      if (p->n_redges == 0) break;
+      cudaMemsetAsync(changed, 0, sizeof(int32_t), st);
+      EAR_LAUNCH(k_cc_hook16, grid_for(p->n_redges), 256, 0, st)(p->re_u, p->re_v, p->n_redges, p->cc, changed);
+      EAR_LAUNCH(k_cc_jump16, grid_for(Np), 256, 0, st)(p->cc, Np);
+      cudaError_t e = cudaMemcpyAsync(&h, changed, sizeof(int32_t), cudaMemcpyDeviceToHost, st);
+      if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+      if (e != cudaSuccess) { set_error("reduced_labels: %s", cudaGetErrorString(e)); s = EAR_ECUDA; }
+      if (!h) break;
+    }
+    cudaFreeAsync(changed, st);
+    EAR_TRY(s);
+  }
+  *out = p->cc;
   return EAR_OK;
 }
 

@@ -36,6 +36,11 @@ cudaEvent_t get_event() {
 
 void count_launch(int n) { g_launches.fetch_add(n, std::memory_order_relaxed); }
 
+void prof_fw16(bool used) {
+  std::lock_guard<std::mutex> lk(g_mu);
+  if (used) g_acc.fw16_used++; else g_acc.fw16_fallbacks++;
+}
+
 int prof_begin(int kind, cudaStream_t s) {
   if (!g_enabled) return -1;
   std::lock_guard<std::mutex> lk(g_mu);
@@ -93,6 +98,11 @@ ear_status_t ear_profile_read(ear_profile_t *out) {
       case PK_SSSP: g_acc.sssp_ms += ms; g_acc.sssp_launches++; g_acc.sssp_arcs += r.work; break;
       case PK_BCC: g_acc.bcc_pieces_ms += ms; break;
       case PK_COMPOSE: g_acc.compose_ms += ms; g_acc.compose_bytes += r.work; break;
+      case PK_FW_P3_16:
+        g_acc.fw_phase3_ms += ms; g_acc.fw_phase3_launches++; g_acc.fw_phase3_minplus += r.work;
+        g_acc.fw_phase3_16_ms += ms; g_acc.fw_phase3_16_minplus += r.work;
+        break;
+      case PK_FW16_CONV: g_acc.fw16_conv_ms += ms; break;
       default: break;
     }
     g_pool.push_back(r.e0);

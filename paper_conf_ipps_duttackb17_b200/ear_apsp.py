@@ -28,6 +28,7 @@ FLAG_NONE = 0
 FLAG_NO_CONTRACT = 1
 FLAG_SSSP = 2
 FLAG_BCC = 4
+FLAG_FW32 = 8
 
 _lib = None
 
@@ -52,7 +53,9 @@ class _Profile(ctypes.Structure):
                 ("same_chain_ms", ctypes.c_double), ("expand_launches", ctypes.c_int64),
                 ("expand_bytes", ctypes.c_double), ("sssp_ms", ctypes.c_double), ("sssp_launches", ctypes.c_int64),
                 ("sssp_arcs", ctypes.c_double), ("bcc_pieces_ms", ctypes.c_double), ("compose_ms", ctypes.c_double),
-                ("compose_bytes", ctypes.c_double)]
+                ("compose_bytes", ctypes.c_double), ("fw16_used", ctypes.c_int64), ("fw16_fallbacks", ctypes.c_int64),
+                ("fw16_conv_ms", ctypes.c_double), ("fw_phase3_16_ms", ctypes.c_double),
+                ("fw_phase3_16_minplus", ctypes.c_double)]
 
 
 class _BccInfo(ctypes.Structure):
