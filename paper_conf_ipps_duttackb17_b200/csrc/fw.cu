@@ -19,6 +19,7 @@
 #include <cudaTypedefs.h>
 
 #include <algorithm>
+#include <cstdlib>
 #include <cmath>
 #include <vector>
 
@@ -509,13 +510,14 @@ struct TileJob16 {
   int64_t ntiles;
 };
 
-template <int KC, int STAGES, int MINB, int UNR>
+template <int KC, int STAGES, int MINB, int UNR, int NTH = 256, int PFC = 0>
 struct Fw16Cfg {
   static constexpr int NCHUNK = TILE / KC;
   static constexpr int A_CHUNK = KC * TILE;   // u16 elements
   static constexpr int B_CHUNK = KC * TILE;   // u32 elements
   static constexpr int SMEM = STAGES * (A_CHUNK * 2 + B_CHUNK * 4) + 2 * STAGES * 8;
-  static constexpr int kKC = KC, kSTAGES = STAGES, kMINB = MINB, kUNR = UNR;
+  static constexpr int kKC = KC, kSTAGES = STAGES, kMINB = MINB, kUNR = UNR, kNTH = NTH, kPFC = PFC;
+  static constexpr int RPH = 256 * 2 / NTH;   // row pairs per 64-row half owned by a thread (2 or 4)
 };
 
 __device__ __forceinline__ void decode16(const TileJob16 &J, int64_t idx, int &ti, int &tj) {
@@ -525,10 +527,13 @@ __device__ __forceinline__ void decode16(const TileJob16 &J, int64_t idx, int &t
   decode_tile(T, idx, ti, tj, lr);
 }
 
+// Thread (ty, tx): columns {tx*4 .. +3, 64 + tx*4 .. +3}; rows {h*64 + ty*2*RPH + 2p, +1} for h = 0, 1 and
+// p < RPH, i.e. 2*RPH row pairs (8 with 256 threads, 16 with 128).
 template <class CF>
-__global__ void __launch_bounds__(NT, CF::kMINB)
+__global__ void __launch_bounds__(CF::kNTH, CF::kMINB)
     k_fw_tiles16(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB, const TileJob16 J) {
-  constexpr int KC = CF::kKC, NCHUNK = CF::NCHUNK, STAGES = CF::kSTAGES;
+  constexpr int KC = CF::kKC, NCHUNK = CF::NCHUNK, STAGES = CF::kSTAGES, NTH = CF::kNTH, RPH = CF::RPH;
+  constexpr int NRP = 2 * RPH;   // row pairs per thread
   extern __shared__ __align__(128) uint8_t smem16[];
   uint16_t *sA = reinterpret_cast<uint16_t *>(smem16);                        // [STAGES][KC][TILE] u16
   uint32_t *sB = reinterpret_cast<uint32_t *>(sA + STAGES * CF::A_CHUNK);     // [STAGES][KC][TILE] u32
@@ -557,7 +562,7 @@ __global__ void __launch_bounds__(NT, CF::kMINB)
   if (tid == 0) {
     for (int s = 0; s < STAGES; ++s) {
       mbar_init(&full[s], 1);
-      mbar_init(&empty[s], NT / 32);
+      mbar_init(&empty[s], NTH / 32);
     }
     asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
     asm volatile("prefetch.tensormap [%0];\n" ::"l"(reinterpret_cast<uint64_t>(&tmA)) : "memory");
@@ -566,15 +571,16 @@ __global__ void __launch_bounds__(NT, CF::kMINB)
   __syncthreads();
   if (tid == 0 && my_tiles > 0) produce(total_chunks < STAGES ? total_chunks : STAGES);
 
+  auto row_of = [&](int r2) { return (r2 < RPH ? 0 : 64) + ty * 2 * RPH + (r2 % RPH) * 2; };
   int g = 0;
   for (int it = 0; it < my_tiles; ++it) {
     int ti, tj;
     tile_of(it, ti, tj);
-    uint32_t c[4][8];
+    uint32_t c[NRP][8];
     uint16_t *Ct = J.C + (int64_t)ti * TILE * J.ldc + (int64_t)tj * TILE;
 #pragma unroll
-    for (int r2 = 0; r2 < 4; ++r2) {
-      const int i = (r2 < 2 ? 0 : 64) + ty * 4 + (r2 & 1) * 2;
+    for (int r2 = 0; r2 < NRP; ++r2) {
+      const int i = row_of(r2);
 #pragma unroll
       for (int h = 0; h < 2; ++h) {
         const uint2 v = *reinterpret_cast<const uint2 *>(Ct + (int64_t)i * J.ldc + h * 64 + tx * 4);
@@ -585,6 +591,14 @@ __global__ void __launch_bounds__(NT, CF::kMINB)
         c[r2][h * 4 + 3] = __byte_perm(v.y, w.y, 0x7632);
       }
     }
+    if (CF::kPFC && it + 1 < my_tiles) {   // pull the next tile's C rows into L2 while this one computes
+      int nti, ntj;
+      tile_of(it + 1, nti, ntj);
+      const uint16_t *Cn = J.C + (int64_t)nti * TILE * J.ldc + (int64_t)ntj * TILE;
+      // 128 rows x 256 B: one 128-byte line per (row, half), spread over the CTA's threads
+      for (int l = tid; l < 2 * TILE; l += NTH)
+        asm volatile("prefetch.global.L2::evict_last [%0];" ::"l"(Cn + (int64_t)(l >> 1) * J.ldc + (l & 1) * 64));
+    }
 #pragma unroll 1
     for (int kc = 0; kc < NCHUNK; ++kc, ++g) {
       if (tid == 0) produce(g + STAGES < total_chunks ? g + STAGES : total_chunks);
@@ -594,14 +608,22 @@ __global__ void __launch_bounds__(NT, CF::kMINB)
       const uint32_t *b_s = sB + st * CF::B_CHUNK;
 #pragma unroll CF::kUNR
       for (int kk = 0; kk < KC; ++kk) {
-        const uint2 alo = *reinterpret_cast<const uint2 *>(a_s + kk * TILE + ty * 4);
-        const uint2 ahi = *reinterpret_cast<const uint2 *>(a_s + kk * TILE + 64 + ty * 4);
+        uint32_t a[NRP];
+        if (RPH == 2) {
+          const uint2 alo = *reinterpret_cast<const uint2 *>(a_s + kk * TILE + ty * 4);
+          const uint2 ahi = *reinterpret_cast<const uint2 *>(a_s + kk * TILE + 64 + ty * 4);
+          a[0] = alo.x; a[1] = alo.y; a[RPH] = ahi.x; a[RPH + 1] = ahi.y;
+        } else {
+          const uint4 alo = *reinterpret_cast<const uint4 *>(a_s + kk * TILE + ty * 8);
+          const uint4 ahi = *reinterpret_cast<const uint4 *>(a_s + kk * TILE + 64 + ty * 8);
+          a[0] = alo.x; a[1] = alo.y; a[2] = alo.z; a[3] = alo.w;
+          a[RPH] = ahi.x; a[RPH + 1] = ahi.y; a[RPH + 2] = ahi.z; a[RPH + 3] = ahi.w;
+        }
         const uint4 blo = *reinterpret_cast<const uint4 *>(b_s + kk * TILE + tx * 4);
         const uint4 bhi = *reinterpret_cast<const uint4 *>(b_s + kk * TILE + 64 + tx * 4);
-        const uint32_t a[4] = {alo.x, alo.y, ahi.x, ahi.y};
         const uint32_t b[8] = {blo.x, blo.y, blo.z, blo.w, bhi.x, bhi.y, bhi.z, bhi.w};
 #pragma unroll
-        for (int r2 = 0; r2 < 4; ++r2)
+        for (int r2 = 0; r2 < NRP; ++r2)
 #pragma unroll
           for (int q = 0; q < 8; ++q) c[r2][q] = __viaddmin_u16x2(a[r2], b[q], c[r2][q]);
       }
@@ -609,8 +631,8 @@ __global__ void __launch_bounds__(NT, CF::kMINB)
       if (lane == 0) mbar_arrive(&empty[st]);
     }
 #pragma unroll
-    for (int r2 = 0; r2 < 4; ++r2) {
-      const int i = (r2 < 2 ? 0 : 64) + ty * 4 + (r2 & 1) * 2;
+    for (int r2 = 0; r2 < NRP; ++r2) {
+      const int i = row_of(r2);
 #pragma unroll
       for (int h = 0; h < 2; ++h) {
         const uint32_t *cc = &c[r2][h * 4];
@@ -625,8 +647,15 @@ __global__ void __launch_bounds__(NT, CF::kMINB)
 #pragma unroll
       for (int q = 0; q < 8; ++q) {
         const int j = (q < 4 ? 0 : 64) + tx * 4 + (q & 3);
-        *reinterpret_cast<uint2 *>(Mt + (int64_t)j * J.ldc + ty * 4) = make_uint2(c[0][q], c[1][q]);
-        *reinterpret_cast<uint2 *>(Mt + (int64_t)j * J.ldc + 64 + ty * 4) = make_uint2(c[2][q], c[3][q]);
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+          if (RPH == 2) {
+            *reinterpret_cast<uint2 *>(Mt + (int64_t)j * J.ldc + h * 64 + ty * 4) = make_uint2(c[h * 2][q], c[h * 2 + 1][q]);
+          } else {
+            *reinterpret_cast<uint4 *>(Mt + (int64_t)j * J.ldc + h * 64 + ty * 8) =
+                make_uint4(c[h * 4][q], c[h * 4 + 1][q], c[h * 4 + 2][q], c[h * 4 + 3][q]);
+          }
+        }
       }
     }
   }
@@ -722,8 +751,37 @@ ear_status_t launch_tiles(const CUtensorMap &map, TileJob J, int64_t nblocks, cu
 }
 
 
-// Packed 16-bit tile kernel configuration: 64-deep k-chunks, 2-stage ring (96 KB), kk unrolled 16x.
-using Fw16Tile = Fw16Cfg<64, 2, 1, 16>;
+// Packed 16-bit tile kernel configuration, chosen by tools/sweep_fw16.py on the B200 (cfg4,
+// profiles/r01_fw16_variants.jsonl): 128 threads with 16 x 8 values each, 32-deep k-chunks, a 2-stage
+// TMA ring (48 KB), 3 CTAs per SM, kk unrolled 16x.  EAR_FW16_VARIANT (development knob) selects one of
+// the measured alternatives below.
+using Fw16Tile = Fw16Cfg<32, 2, 3, 16, 128>;
+using Fw16V0 = Fw16Cfg<64, 2, 1, 16>;
+using Fw16V1 = Fw16Cfg<64, 2, 2, 16>;
+using Fw16V2 = Fw16Cfg<32, 3, 2, 16>;
+using Fw16V3 = Fw16Cfg<32, 2, 2, 16>;
+using Fw16V4 = Fw16Cfg<64, 3, 1, 16>;
+using Fw16V5 = Fw16Cfg<32, 4, 2, 8>;
+using Fw16V6 = Fw16Cfg<64, 2, 2, 8>;
+using Fw16V7 = Fw16Cfg<32, 2, 4, 8, 128>;
+using Fw16V8 = Fw16Cfg<64, 2, 2, 8, 128>;
+using Fw16V9 = Fw16Cfg<32, 3, 3, 8, 128>;
+using Fw16V10 = Fw16Cfg<32, 2, 3, 16, 128>;
+using Fw16V11 = Fw16Cfg<32, 2, 3, 16, 128, 1>;
+using Fw16V12 = Fw16Cfg<64, 2, 1, 16, 256, 1>;
+using Fw16V13 = Fw16Cfg<32, 3, 2, 16, 128, 1>;
+using Fw16V14 = Fw16Cfg<16, 4, 3, 16, 128>;
+using Fw16V15 = Fw16Cfg<16, 6, 3, 16, 128>;
+using Fw16V16 = Fw16Cfg<32, 3, 3, 16, 128>;
+int fw16_variant() {
+  static int v = -1;
+  if (v < 0) {
+    const char *e = getenv("EAR_FW16_VARIANT");
+    v = e ? atoi(e) : -1;
+    if (v < 0) v = 99;   // the default configuration
+  }
+  return v;
+}
 
 template <class CF>
 ear_status_t launch16(const CUtensorMap &mA, const CUtensorMap &mB, TileJob16 J, int64_t nblocks, cudaStream_t st) {
@@ -734,11 +792,11 @@ ear_status_t launch16(const CUtensorMap &mA, const CUtensorMap &mB, TileJob16 J,
     attr = true;
   }
   int per_sm = 0;
-  EAR_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_fw_tiles16<CF>, NT, CF::SMEM));
+  EAR_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_fw_tiles16<CF>, CF::kNTH, CF::SMEM));
   if (per_sm < 1) per_sm = 1;
   J.ntiles = nblocks;
   const int64_t grid = std::min<int64_t>(nblocks, (int64_t)g_num_sms * per_sm);
-  EAR_LAUNCH(k_fw_tiles16<CF>, (unsigned)grid, NT, CF::SMEM, st)(mA, mB, J);
+  EAR_LAUNCH(k_fw_tiles16<CF>, (unsigned)grid, CF::kNTH, CF::SMEM, st)(mA, mB, J);
   return EAR_OK;
 }
 
@@ -767,10 +825,34 @@ ear_status_t fw_single16(int32_t *D, int64_t ldd, int32_t Np, const int32_t *lab
     if (Pd) cudaFreeAsync(Pd, st);
     return EAR_OK;   // no room for the 16-bit copy: the int32 path runs
   }
+  const int var = fw16_variant();
+  const int kc16 = (var == 14 || var == 15) ? 16 : (var == 99 || var == 2 || var == 3 || var == 5 || var == 7 || var == 9 || var == 10 || var == 11 || var == 13 || var == 16) ? 32 : 64;
   ear_status_t s = EAR_OK;
   CUtensorMap mA, mB;
-  s = make_map_t(&mA, CU_TENSOR_MAP_DATA_TYPE_UINT16, 2, D16, Np, Np, Np, Fw16Tile::kKC);
-  if (s == EAR_OK) s = make_map_t(&mB, CU_TENSOR_MAP_DATA_TYPE_UINT32, 4, Pd, TILE, Np, Np, Fw16Tile::kKC);
+  s = make_map_t(&mA, CU_TENSOR_MAP_DATA_TYPE_UINT16, 2, D16, Np, Np, Np, kc16);
+  auto run16 = [&](const TileJob16 &J, int64_t nb) -> ear_status_t {
+    switch (var) {
+      case 1: return launch16<Fw16V1>(mA, mB, J, nb, st);
+      case 2: return launch16<Fw16V2>(mA, mB, J, nb, st);
+      case 3: return launch16<Fw16V3>(mA, mB, J, nb, st);
+      case 4: return launch16<Fw16V4>(mA, mB, J, nb, st);
+      case 5: return launch16<Fw16V5>(mA, mB, J, nb, st);
+      case 6: return launch16<Fw16V6>(mA, mB, J, nb, st);
+      case 7: return launch16<Fw16V7>(mA, mB, J, nb, st);
+      case 8: return launch16<Fw16V8>(mA, mB, J, nb, st);
+      case 9: return launch16<Fw16V9>(mA, mB, J, nb, st);
+      case 10: return launch16<Fw16V10>(mA, mB, J, nb, st);
+      case 11: return launch16<Fw16V11>(mA, mB, J, nb, st);
+      case 12: return launch16<Fw16V12>(mA, mB, J, nb, st);
+      case 13: return launch16<Fw16V13>(mA, mB, J, nb, st);
+      case 14: return launch16<Fw16V14>(mA, mB, J, nb, st);
+      case 15: return launch16<Fw16V15>(mA, mB, J, nb, st);
+      case 16: return launch16<Fw16V16>(mA, mB, J, nb, st);
+      case 0: return launch16<Fw16V0>(mA, mB, J, nb, st);
+      default: return launch16<Fw16Tile>(mA, mB, J, nb, st);
+    }
+  };
+  if (s == EAR_OK) s = make_map_t(&mB, CU_TENSOR_MAP_DATA_TYPE_UINT32, 4, Pd, TILE, Np, Np, kc16);
   const int64_t ndup = (int64_t)TILE * (Np / 4);
   if (s == EAR_OK) {
     int sc = prof_begin(PK_FW16_CONV, st);
@@ -785,14 +867,14 @@ ear_status_t fw_single16(int32_t *D, int64_t ldd, int32_t Np, const int32_t *lab
     int s2 = prof_begin(PK_FW_P2, st);
     EAR_LAUNCH(k_dup16, grid_for(ndup), 256, 0, st)(P16, Np, Pd);
     TileJob16 J{D16, Np, k * TILE, k, nt, MODE_PIVOT_ROW, 1, 0};
-    s = launch16<Fw16Tile>(mA, mB, J, nt - 1, st);
+    s = run16(J, nt - 1);
     if (s == EAR_OK) EAR_LAUNCH(k_dup16, grid_for(ndup), 256, 0, st)(P16, Np, Pd);
     prof_end(s2, st, (nt - 1) * tile_ops);
     if (s != EAR_OK) break;
     J.mode = MODE_UPPER;
     const int64_t nup = (int64_t)(nt - 1) * nt / 2;
     int s3 = prof_begin(PK_FW_P3_16, st);
-    s = launch16<Fw16Tile>(mA, mB, J, nup, st);
+    s = run16(J, nup);
     prof_end(s3, st, nup * tile_ops);
   }
   int32_t h_bad = 1;

@@ -1,5 +1,8 @@
-# ncu captures of the two dominant kernels on cfg4 (one bench step, no warm-up), plus the host timeline
+# Round profile set on cfg4: bench line, ncu launch list of one step, ncu --set full of the top kernels.
 TAG=${1:-r01}
-python tools/host_timeline.py cfg4 2>&1 | tail -5
-timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_fw_tiles -s 21 -c 1 -o gpurun_out/prof_fw_$TAG python bench.py --steps 1 --warmup 0 --no-e2e --no-cpu-baseline > /dev/null 2> gpurun_out/ncu_fw_$TAG.log; tail -1 gpurun_out/ncu_fw_$TAG.log
-timeout 600 ncu --set full --clock-control none --import-source on -k regex:k_expand -c 1 -o gpurun_out/prof_expand_$TAG python bench.py --steps 1 --warmup 0 --no-e2e --no-cpu-baseline > /dev/null 2> gpurun_out/ncu_ex_$TAG.log; tail -1 gpurun_out/ncu_ex_$TAG.log
+set -x
+timeout 900 python bench.py > gpurun_out/bench_$TAG.json 2> gpurun_out/bench_$TAG.log; tail -2 gpurun_out/bench_$TAG.log; cat gpurun_out/bench_$TAG.json
+timeout 1200 ncu --metrics gpu__time_duration.sum --clock-control none -c 8000 --csv --log-file gpurun_out/launches_$TAG.csv python bench.py --steps 1 --warmup 0 --no-e2e --no-cpu-baseline --no-alt > /dev/null 2> gpurun_out/ncu_launch_$TAG.log; tail -1 gpurun_out/ncu_launch_$TAG.log
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_fw_tiles16 -s 101 -c 1 -o gpurun_out/prof_fw16_$TAG python bench.py --steps 1 --warmup 0 --no-e2e --no-cpu-baseline --no-alt > /dev/null 2> gpurun_out/ncu_fw_$TAG.log; tail -1 gpurun_out/ncu_fw_$TAG.log
+timeout 600 ncu --set full --clock-control none --import-source on -k regex:k_expand -c 1 -o gpurun_out/prof_expand_$TAG python bench.py --steps 1 --warmup 0 --no-e2e --no-cpu-baseline --no-alt > /dev/null 2> gpurun_out/ncu_ex_$TAG.log; tail -1 gpurun_out/ncu_ex_$TAG.log
+ls -la gpurun_out
