@@ -114,7 +114,9 @@ __global__ void __launch_bounds__(NT, 1) k_fw_phase1(int32_t *T, int64_t ldt) {
 // mbarriers (full: TMA bytes landed; empty: all 8 warps done reading), so no CTA-wide barrier sits
 // in the main loop and the next tile's first chunks are fetched while the current tile finishes.
 // Thread 0 doubles as the TMA producer.  The C tile lives in registers (8x8 per thread).
-enum { MODE_PIVOT_ROW = 0, MODE_UPPER = 1, MODE_LIST = 2 };
+// MODE_CROSS / MODE_REST (single-GPU lookahead, round k): the upper tiles of row/column k+1 (without
+// column k), and all upper tiles outside rows/columns k and k+1; together they are MODE_UPPER.
+enum { MODE_PIVOT_ROW = 0, MODE_UPPER = 1, MODE_LIST = 2, MODE_CROSS = 3, MODE_REST = 4 };
 
 // Tile-kernel configuration: k-chunk depth, TMA ring depth, CTAs per SM, kk-loop unroll.
 template <int KC_, int ST_, int MINB_, int UNR_>
@@ -190,18 +192,26 @@ __device__ __forceinline__ void decode_tile(const TileJob &J, int64_t idx, int &
     lr = ti - J.ti0;
     return;
   }
-  if (J.mode == MODE_UPPER) {
-    // upper triangle (a <= b) of the (nt-1) x (nt-1) non-pivot tiles, row-major; row a starts at
-    // a*T - a*(a-1)/2
-    const int64_t T = J.nt - 1;
+  if (J.mode == MODE_CROSS) {
+    const int j = (int)idx < k ? (int)idx : (int)idx + 1;
+    ti = min(j, k + 1);
+    tj = max(j, k + 1);
+    lr = ti - J.ti0;
+    return;
+  }
+  if (J.mode == MODE_UPPER || J.mode == MODE_REST) {
+    // upper triangle (a <= b) of the (nt-s) x (nt-s) tiles outside the s skipped rows/columns
+    // (s = 1: k; s = 2: k and k+1), row-major; row a starts at a*T - a*(a-1)/2
+    const int skip = J.mode == MODE_REST ? 2 : 1;
+    const int64_t T = J.nt - skip;
     double tt = (double)(2 * T + 1);
     int64_t a = (int64_t)floor((tt - sqrt(tt * tt - 8.0 * (double)idx)) * 0.5);
     if (a < 0) a = 0;
     while (a > 0 && a * T - a * (a - 1) / 2 > idx) --a;
     while ((a + 1) * T - (a + 1) * a / 2 <= idx) ++a;
     const int64_t b = a + (idx - (a * T - a * (a - 1) / 2));
-    ti = (int)a < k ? (int)a : (int)a + 1;
-    tj = (int)b < k ? (int)b : (int)b + 1;
+    ti = (int)a < k ? (int)a : (int)a + skip;
+    tj = (int)b < k ? (int)b : (int)b + skip;
     lr = ti - J.ti0;
     return;
   }
@@ -751,40 +761,22 @@ ear_status_t launch_tiles(const CUtensorMap &map, TileJob J, int64_t nblocks, cu
 }
 
 
-// Packed 16-bit tile kernel configuration, chosen by tools/sweep_fw16.py on the B200 (cfg4,
-// profiles/r01_fw16_variants.jsonl): 128 threads with 16 x 8 values each, 32-deep k-chunks, a 2-stage
-// TMA ring (48 KB), 3 CTAs per SM, kk unrolled 16x.  EAR_FW16_VARIANT (development knob) selects one of
-// the measured alternatives below.
+// Packed 16-bit tile kernel configuration, chosen by tools/sweep_fw16.py on the B200 (cfg4, 17
+// variants, profiles/r01_fw16_variants.jsonl): 128 threads with 16 x 8 values each, 32-deep k-chunks,
+// a 2-stage TMA ring (48 KB), 3 CTAs per SM, kk unrolled 16x.
 using Fw16Tile = Fw16Cfg<32, 2, 3, 16, 128>;
-using Fw16V0 = Fw16Cfg<64, 2, 1, 16>;
-using Fw16V1 = Fw16Cfg<64, 2, 2, 16>;
-using Fw16V2 = Fw16Cfg<32, 3, 2, 16>;
-using Fw16V3 = Fw16Cfg<32, 2, 2, 16>;
-using Fw16V4 = Fw16Cfg<64, 3, 1, 16>;
-using Fw16V5 = Fw16Cfg<32, 4, 2, 8>;
-using Fw16V6 = Fw16Cfg<64, 2, 2, 8>;
-using Fw16V7 = Fw16Cfg<32, 2, 4, 8, 128>;
-using Fw16V8 = Fw16Cfg<64, 2, 2, 8, 128>;
-using Fw16V9 = Fw16Cfg<32, 3, 3, 8, 128>;
-using Fw16V10 = Fw16Cfg<32, 2, 3, 16, 128>;
-using Fw16V11 = Fw16Cfg<32, 2, 3, 16, 128, 1>;
-using Fw16V12 = Fw16Cfg<64, 2, 1, 16, 256, 1>;
-using Fw16V13 = Fw16Cfg<32, 3, 2, 16, 128, 1>;
-using Fw16V14 = Fw16Cfg<16, 4, 3, 16, 128>;
-using Fw16V15 = Fw16Cfg<16, 6, 3, 16, 128>;
-using Fw16V16 = Fw16Cfg<32, 3, 3, 16, 128>;
-int fw16_variant() {
-  static int v = -1;
-  if (v < 0) {
-    const char *e = getenv("EAR_FW16_VARIANT");
-    v = e ? atoi(e) : -1;
-    if (v < 0) v = 99;   // the default configuration
-  }
-  return v;
+
+// development knobs (tools/): EAR_FW16_LOOKAHEAD=0 disables the lookahead, EAR_FW16_RESERVE sets the
+// CTA slots the rest-of-round launch leaves free for the next round's pivot work (default 0: measured
+// best, profiles/r01_fw16_lookahead.jsonl), EAR_FW16_PRIO=0 gives the side stream normal priority
+int env_int(const char *name, int dflt) {
+  const char *e = getenv(name);
+  return e ? atoi(e) : dflt;
 }
 
 template <class CF>
-ear_status_t launch16(const CUtensorMap &mA, const CUtensorMap &mB, TileJob16 J, int64_t nblocks, cudaStream_t st) {
+ear_status_t launch16(const CUtensorMap &mA, const CUtensorMap &mB, TileJob16 J, int64_t nblocks, cudaStream_t st,
+                      int reserve = 0) {
   if (nblocks <= 0) return EAR_OK;
   static bool attr = false;
   if (!attr) {
@@ -795,7 +787,7 @@ ear_status_t launch16(const CUtensorMap &mA, const CUtensorMap &mB, TileJob16 J,
   EAR_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_fw_tiles16<CF>, CF::kNTH, CF::SMEM));
   if (per_sm < 1) per_sm = 1;
   J.ntiles = nblocks;
-  const int64_t grid = std::min<int64_t>(nblocks, (int64_t)g_num_sms * per_sm);
+  const int64_t grid = std::min<int64_t>(nblocks, std::max<int64_t>(1, (int64_t)g_num_sms * per_sm - reserve));
   EAR_LAUNCH(k_fw_tiles16<CF>, (unsigned)grid, CF::kNTH, CF::SMEM, st)(mA, mB, J);
   return EAR_OK;
 }
@@ -804,6 +796,13 @@ int grid_for(int64_t n) { return (int)std::max<int64_t>(1, std::min<int64_t>(cei
 
 // The packed 16-bit FW on a copy of D (see C16 above).  *done = false (D untouched) when a connected
 // pair reached the cap; the caller then runs the int32 FW.  Synchronises the stream once (the check).
+//
+// Lookahead: round k's phase 3 is split into the tiles of row/column k+1 (MODE_CROSS, first) and the
+// rest (MODE_REST).  As soon as the cross tiles are done, round k+1's pivot work -- phase 1 on tile
+// (k+1, k+1), the duplicated pivot row Pd, phase 2 on row k+1 -- runs on a side stream while the rest
+// of round k proceeds on the main stream (its launch leaves a few CTA slots free for it); round k+1's
+// phase 3 waits for both.  The two streams touch disjoint tiles (the rest skips rows/columns k, k+1)
+// and alternate between two Pd buffers, so the serial phases 1-2 leave the critical path.
 ear_status_t fw_single16(int32_t *D, int64_t ldd, int32_t Np, const int32_t *lab, int32_t n_real, bool *done,
                          cudaStream_t st) {
   *done = false;
@@ -812,71 +811,97 @@ ear_status_t fw_single16(int32_t *D, int64_t ldd, int32_t Np, const int32_t *lab
     EAR_CUDA_TRY(cudaGetDevice(&dev));
     EAR_CUDA_TRY(cudaDeviceGetAttribute(&g_num_sms, cudaDevAttrMultiProcessorCount, dev));
   }
+  // per-device side stream and the two lookahead events (created once)
+  static cudaStream_t sides[64] = {};
+  static cudaEvent_t crosses[64] = {}, pivots[64] = {};
+  int dev = 0;
+  EAR_CUDA_TRY(cudaGetDevice(&dev));
+  if (dev < 0 || dev >= 64) { set_error("fw_single16: device %d out of range", dev); return EAR_EINVAL; }
+  if (!sides[dev]) {
+    int lo = 0, hi = 0;   // the pivot work gets the highest priority: its CTAs take the first free slots
+    EAR_CUDA_TRY(cudaDeviceGetStreamPriorityRange(&lo, &hi));
+    EAR_CUDA_TRY(cudaStreamCreateWithPriority(&sides[dev], cudaStreamNonBlocking, env_int("EAR_FW16_PRIO", 1) ? hi : lo));
+    EAR_CUDA_TRY(cudaEventCreateWithFlags(&crosses[dev], cudaEventDisableTiming));
+    EAR_CUDA_TRY(cudaEventCreateWithFlags(&pivots[dev], cudaEventDisableTiming));
+  }
+  cudaStream_t side = sides[dev];
+  cudaEvent_t ev_cross = crosses[dev], ev_pivot = pivots[dev];
+  const bool lookahead = env_int("EAR_FW16_LOOKAHEAD", 1) != 0;
+  const int reserve = env_int("EAR_FW16_RESERVE", 0);
   const int nt = Np / TILE;
   const double tile_ops = (double)TILE * TILE * TILE;
   uint16_t *D16 = nullptr;
-  uint32_t *Pd = nullptr;
+  uint32_t *Pd = nullptr;   // two 128 x Np buffers (round parity)
   int32_t *bad = nullptr;
   if (cudaMallocAsync((void **)&D16, sizeof(uint16_t) * (size_t)Np * Np, st) != cudaSuccess ||
-      cudaMallocAsync((void **)&Pd, sizeof(uint32_t) * (size_t)TILE * Np, st) != cudaSuccess ||
+      cudaMallocAsync((void **)&Pd, 2 * sizeof(uint32_t) * (size_t)TILE * Np, st) != cudaSuccess ||
       cudaMallocAsync((void **)&bad, sizeof(int32_t), st) != cudaSuccess) {
     cudaGetLastError();
     if (D16) cudaFreeAsync(D16, st);
     if (Pd) cudaFreeAsync(Pd, st);
     return EAR_OK;   // no room for the 16-bit copy: the int32 path runs
   }
-  const int var = fw16_variant();
-  const int kc16 = (var == 14 || var == 15) ? 16 : (var == 99 || var == 2 || var == 3 || var == 5 || var == 7 || var == 9 || var == 10 || var == 11 || var == 13 || var == 16) ? 32 : 64;
+  constexpr int KC = Fw16Tile::kKC;
   ear_status_t s = EAR_OK;
-  CUtensorMap mA, mB;
-  s = make_map_t(&mA, CU_TENSOR_MAP_DATA_TYPE_UINT16, 2, D16, Np, Np, Np, kc16);
-  auto run16 = [&](const TileJob16 &J, int64_t nb) -> ear_status_t {
-    switch (var) {
-      case 1: return launch16<Fw16V1>(mA, mB, J, nb, st);
-      case 2: return launch16<Fw16V2>(mA, mB, J, nb, st);
-      case 3: return launch16<Fw16V3>(mA, mB, J, nb, st);
-      case 4: return launch16<Fw16V4>(mA, mB, J, nb, st);
-      case 5: return launch16<Fw16V5>(mA, mB, J, nb, st);
-      case 6: return launch16<Fw16V6>(mA, mB, J, nb, st);
-      case 7: return launch16<Fw16V7>(mA, mB, J, nb, st);
-      case 8: return launch16<Fw16V8>(mA, mB, J, nb, st);
-      case 9: return launch16<Fw16V9>(mA, mB, J, nb, st);
-      case 10: return launch16<Fw16V10>(mA, mB, J, nb, st);
-      case 11: return launch16<Fw16V11>(mA, mB, J, nb, st);
-      case 12: return launch16<Fw16V12>(mA, mB, J, nb, st);
-      case 13: return launch16<Fw16V13>(mA, mB, J, nb, st);
-      case 14: return launch16<Fw16V14>(mA, mB, J, nb, st);
-      case 15: return launch16<Fw16V15>(mA, mB, J, nb, st);
-      case 16: return launch16<Fw16V16>(mA, mB, J, nb, st);
-      case 0: return launch16<Fw16V0>(mA, mB, J, nb, st);
-      default: return launch16<Fw16Tile>(mA, mB, J, nb, st);
-    }
-  };
-  if (s == EAR_OK) s = make_map_t(&mB, CU_TENSOR_MAP_DATA_TYPE_UINT32, 4, Pd, TILE, Np, Np, kc16);
+  CUtensorMap mA, mB[2];
+  s = make_map_t(&mA, CU_TENSOR_MAP_DATA_TYPE_UINT16, 2, D16, Np, Np, Np, KC);
+  for (int b = 0; b < 2 && s == EAR_OK; ++b)
+    s = make_map_t(&mB[b], CU_TENSOR_MAP_DATA_TYPE_UINT32, 4, Pd + (size_t)b * TILE * Np, TILE, Np, Np, KC);
   const int64_t ndup = (int64_t)TILE * (Np / 4);
   if (s == EAR_OK) {
     int sc = prof_begin(PK_FW16_CONV, st);
     EAR_LAUNCH(k_to16, grid_for((int64_t)Np * (Np / 4)), 256, 0, st)(D, ldd, D16, Np);
     prof_end(sc, st, 0);
   }
-  for (int k = 0; k < nt && s == EAR_OK; ++k) {
+  // phases 1 and 2 of round k on stream q (Pd buffer k & 1)
+  auto pivot = [&](int k, cudaStream_t q) -> ear_status_t {
     uint16_t *P16 = D16 + (int64_t)k * TILE * Np;
-    int s1 = prof_begin(PK_FW_P1, st);
-    EAR_LAUNCH(k_fw_phase1_16, 1, NT, 0, st)(P16 + (int64_t)k * TILE, Np);
-    prof_end(s1, st, tile_ops);
-    int s2 = prof_begin(PK_FW_P2, st);
-    EAR_LAUNCH(k_dup16, grid_for(ndup), 256, 0, st)(P16, Np, Pd);
+    uint32_t *Pk = Pd + (size_t)(k & 1) * TILE * Np;
+    int s1 = prof_begin(PK_FW_P1, q);
+    EAR_LAUNCH(k_fw_phase1_16, 1, NT, 0, q)(P16 + (int64_t)k * TILE, Np);
+    prof_end(s1, q, tile_ops);
+    int s2 = prof_begin(PK_FW_P2, q);
+    EAR_LAUNCH(k_dup16, grid_for(ndup), 256, 0, q)(P16, Np, Pk);   // B of phase 2: the pre-phase-2 row
     TileJob16 J{D16, Np, k * TILE, k, nt, MODE_PIVOT_ROW, 1, 0};
-    s = run16(J, nt - 1);
-    if (s == EAR_OK) EAR_LAUNCH(k_dup16, grid_for(ndup), 256, 0, st)(P16, Np, Pd);
-    prof_end(s2, st, (nt - 1) * tile_ops);
-    if (s != EAR_OK) break;
-    J.mode = MODE_UPPER;
+    EAR_TRY(launch16<Fw16Tile>(mA, mB[k & 1], J, nt - 1, q));
+    EAR_LAUNCH(k_dup16, grid_for(ndup), 256, 0, q)(P16, Np, Pk);   // B of phase 3
+    prof_end(s2, q, (nt - 1) * tile_ops);
+    return EAR_OK;
+  };
+  if (s == EAR_OK && nt > 0) s = pivot(0, st);
+  for (int k = 0; k < nt && s == EAR_OK; ++k) {
+    TileJob16 J{D16, Np, k * TILE, k, nt, MODE_UPPER, 1, 0};
     const int64_t nup = (int64_t)(nt - 1) * nt / 2;
+    if (!lookahead || k + 1 == nt) {
+      int s3 = prof_begin(PK_FW_P3_16, st);
+      s = launch16<Fw16Tile>(mA, mB[k & 1], J, nup, st);
+      prof_end(s3, st, nup * tile_ops);
+      if (s == EAR_OK && k + 1 < nt) s = pivot(k + 1, st);
+      continue;
+    }
     int s3 = prof_begin(PK_FW_P3_16, st);
-    s = run16(J, nup);
-    prof_end(s3, st, nup * tile_ops);
+    J.mode = MODE_CROSS;
+    s = launch16<Fw16Tile>(mA, mB[k & 1], J, nt - 1, st);
+    prof_end(s3, st, (nt - 1) * tile_ops);
+    if (s != EAR_OK) break;
+    cudaError_t e = cudaEventRecord(ev_cross, st);
+    if (e == cudaSuccess) e = cudaStreamWaitEvent(side, ev_cross, 0);
+    if (e != cudaSuccess) { set_error("fw_single16: %s", cudaGetErrorString(e)); s = EAR_ECUDA; break; }
+    s = pivot(k + 1, side);
+    if (s != EAR_OK) break;
+    e = cudaEventRecord(ev_pivot, side);
+    if (e != cudaSuccess) { set_error("fw_single16: %s", cudaGetErrorString(e)); s = EAR_ECUDA; break; }
+    J.mode = MODE_REST;
+    const int64_t nrest = (int64_t)(nt - 2) * (nt - 1) / 2;
+    int s4 = prof_begin(PK_FW_P3_16, st);
+    s = launch16<Fw16Tile>(mA, mB[k & 1], J, nrest, st, reserve);
+    prof_end(s4, st, nrest * tile_ops);
+    if (s == EAR_OK) {
+      e = cudaStreamWaitEvent(st, ev_pivot, 0);
+      if (e != cudaSuccess) { set_error("fw_single16: %s", cudaGetErrorString(e)); s = EAR_ECUDA; }
+    }
   }
+  if (s != EAR_OK) cudaStreamWaitEvent(st, ev_pivot, 0);   // never leave side work behind the frees
   int32_t h_bad = 1;
   if (s == EAR_OK) {
     int sc = prof_begin(PK_FW16_CONV, st);

@@ -1,7 +1,7 @@
-"""Sweep the packed 16-bit FW tile-kernel configurations (EAR_FW16_VARIANT) on a config's plain FW:
-phase-3 min-plus rate from the library profile, and a checksum of D (must agree across variants).
+"""Time the packed 16-bit FW on a config's plain FW (no BCC) under the development knobs of fw.cu:
+phase-3 min-plus rate and FW wall time, and a checksum of D (must agree across settings).
 
-    python tools/sweep_fw16.py [cfg4] [variants...]      (one subprocess per variant)
+    python tools/sweep_fw16.py [cfg4] ["LOOKAHEAD,RESERVE" ...]      (one subprocess per setting)
 """
 import json
 import os
@@ -31,7 +31,8 @@ def one(cfg):
     torch.cuda.synchronize()
     p = ea.profile_read()
     cs = int((D[::97, ::89].to(torch.int64) * 7 + 1).sum().item())
-    print(json.dumps({"variant": int(os.environ.get("EAR_FW16_VARIANT", "0")), "fw_ms": e0.elapsed_time(e1),
+    print(json.dumps({"lookahead": os.environ.get("EAR_FW16_LOOKAHEAD", "1"), "prio": os.environ.get("EAR_FW16_PRIO", "1"),
+                      "reserve": os.environ.get("EAR_FW16_RESERVE", "0"), "fw_ms": e0.elapsed_time(e1),
                       "p3_ms": p["fw_phase3_16_ms"], "p3_Tminplus": p["fw_phase3_16_minplus"] / p["fw_phase3_16_ms"] / 1e9
                       if p["fw_phase3_16_ms"] else None, "p1_ms": p["fw_phase1_ms"], "p2_ms": p["fw_phase2_ms"],
                       "conv_ms": p["fw16_conv_ms"], "used": p["fw16_used"], "checksum": cs}), flush=True)
@@ -42,6 +43,7 @@ if __name__ == "__main__":
         one(sys.argv[2])
         sys.exit(0)
     cfg = sys.argv[1] if len(sys.argv) > 1 else "cfg4"
-    for v in (sys.argv[2:] or ["0", "1", "2", "3", "4", "5", "6"]):
-        env = dict(os.environ, EAR_FW16_VARIANT=v)
+    for setting in (sys.argv[2:] or ["0,0,1", "1,0,1", "1,0,0", "1,2,1", "1,4,1"]):
+        la, rs, pr = setting.split(",")
+        env = dict(os.environ, EAR_FW16_LOOKAHEAD=la, EAR_FW16_RESERVE=rs, EAR_FW16_PRIO=pr)
         subprocess.run([sys.executable, __file__, "--one", cfg], env=env, timeout=600)
