@@ -663,7 +663,6 @@ ear_status_t bcc_prepare(ear_plan_s *p, int32_t P, cudaStream_t st) {
   return EAR_OK;
 }
 
-ear_status_t fw_sharded(int32_t *S, int64_t ldd, int32_t Np, ear_comm_s *comm, cudaStream_t st);
 ear_status_t fw_sharded_gather(const int32_t *S, int64_t ldd, int32_t Np, int32_t *Df, int64_t ldf, ear_comm_s *comm,
                                cudaStream_t st);
 std::vector<int32_t> shard_rows(int32_t nt, int32_t P, int32_t rank);
@@ -712,7 +711,8 @@ ear_status_t bcc_solve(ear_plan_s *p, ear_comm_s *comm, int32_t *D, int64_t ldd,
         if (cudaMemcpyAsync(S + (int64_t)j * TILE * ld, M + (int64_t)own[j] * TILE * ld,
                             sizeof(int32_t) * (size_t)TILE * ld, cudaMemcpyDeviceToDevice, st) != cudaSuccess)
           s = EAR_ECUDA;
-      if (s == EAR_OK) s = fw_sharded(S, ld, ld, comm, st);
+      if (s == EAR_OK)   // a piece is connected: no labels
+        s = fw_sharded_auto(S, ld, ld, comm, nullptr, b->h_psize[id], !(p->flags & EAR_FLAG_FW32), st);
       if (s == EAR_OK) s = fw_sharded_gather(S, ld, ld, M, ld, comm, st);
       cudaFreeAsync(S, st);
     } else {

@@ -452,6 +452,108 @@ __global__ void k_dup16(const uint16_t *__restrict__ P16, int32_t Np, uint32_t *
   }
 }
 
+// ---- 16-bit row-block sharding (fw_sharded16 below)
+// rows x cols block of int32 (ld lds) -> capped u16 (ld ld16); cols % 4 == 0
+__global__ void k_to16r(const int32_t *__restrict__ S, int64_t lds, uint16_t *__restrict__ S16, int64_t ld16,
+                        int64_t rows, int32_t cols) {
+  const int64_t total = rows * (cols / 4);
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t r = i / (cols / 4);
+    const int32_t c4 = (int32_t)(i % (cols / 4)) * 4;
+    const int4 v = *reinterpret_cast<const int4 *>(S + r * lds + c4);
+    const uint32_t lo = (uint32_t)min(v.x, (int32_t)C16) | ((uint32_t)min(v.y, (int32_t)C16) << 16);
+    const uint32_t hi = (uint32_t)min(v.z, (int32_t)C16) | ((uint32_t)min(v.w, (int32_t)C16) << 16);
+    *reinterpret_cast<uint2 *>(S16 + r * ld16 + c4) = make_uint2(lo, hi);
+  }
+}
+
+// the inverse (C16 -> INF)
+__global__ void k_from16r(const uint16_t *__restrict__ S16, int64_t ld16, int32_t *__restrict__ S, int64_t lds,
+                          int64_t rows, int32_t cols) {
+  const int64_t total = rows * (cols / 4);
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t r = i / (cols / 4);
+    const int32_t c4 = (int32_t)(i % (cols / 4)) * 4;
+    const uint2 v = *reinterpret_cast<const uint2 *>(S16 + r * ld16 + c4);
+    auto f = [](uint32_t x) { return x == C16 ? INF : (int32_t)x; };
+    *reinterpret_cast<int4 *>(S + r * lds + c4) = make_int4(f(v.x & 0xFFFFu), f(v.x >> 16), f(v.y & 0xFFFFu), f(v.y >> 16));
+  }
+}
+
+// k_prow_xfer for a 16-bit owned storage: dir 0 gathers S16 pieces into the int32 exchange block
+// (u16 -> int32; C16 < INF, so the MIN all-reduce keeps it), dir 1 scatters the capped 16-bit pivot
+// row block back.  Same grid and piece rule as k_prow_xfer.
+template <class TP>
+__global__ void k_prow_xfer16(uint16_t *S, int64_t ldd, const int32_t *orow, int32_t k, TP *prow, int32_t Np, int dir) {
+  __shared__ uint32_t t[32][33];
+  const int lr = blockIdx.z, ti = orow[lr], tj = blockIdx.y;
+  const int bx = blockIdx.x & 3, by = blockIdx.x >> 2;
+  const int lx = threadIdx.x & 31, ly = threadIdx.x >> 5;
+  if (ti == k) {
+    if (tj < k) return;
+    for (int yy = ly; yy < 32; yy += 8) {
+      const int64_t row = by * 32 + yy, col = (int64_t)tj * TILE + bx * 32 + lx;
+      uint16_t *s = S + ((int64_t)lr * TILE + row) * ldd + col;
+      TP *p = prow + row * Np + col;
+      if (dir == 0) *p = (TP)*s; else *s = (uint16_t)*p;
+    }
+    return;
+  }
+  if (ti > k || tj != k) return;
+  if (dir == 0) {
+    for (int yy = ly; yy < 32; yy += 8)
+      t[yy][lx] = S[((int64_t)lr * TILE + bx * 32 + yy) * ldd + (int64_t)k * TILE + by * 32 + lx];
+    __syncthreads();
+    for (int yy = ly; yy < 32; yy += 8)
+      prow[(int64_t)(by * 32 + yy) * Np + (int64_t)ti * TILE + bx * 32 + lx] = (TP)t[lx][yy];
+  } else {
+    for (int yy = ly; yy < 32; yy += 8)
+      t[yy][lx] = (uint32_t)prow[(int64_t)(by * 32 + yy) * Np + (int64_t)ti * TILE + bx * 32 + lx];
+    __syncthreads();
+    for (int yy = ly; yy < 32; yy += 8)
+      S[((int64_t)lr * TILE + bx * 32 + yy) * ldd + (int64_t)k * TILE + by * 32 + lx] = (uint16_t)t[lx][yy];
+  }
+}
+
+// the pivot row block after the int32 phases 1-2 -> its capped u16 copy (A operand, scattered back to
+// the owners) and the duplicated u32 copy (B operand); n = TILE * Np, n % 4 == 0
+__global__ void k_prow_to16(const int32_t *__restrict__ P32, uint16_t *__restrict__ P16, uint32_t *__restrict__ Pd,
+                            int64_t n) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n / 4; i += (int64_t)gridDim.x * blockDim.x) {
+    const int4 v = reinterpret_cast<const int4 *>(P32)[i];
+    const uint32_t a = (uint32_t)min(v.x, (int32_t)C16), b = (uint32_t)min(v.y, (int32_t)C16);
+    const uint32_t c = (uint32_t)min(v.z, (int32_t)C16), d = (uint32_t)min(v.w, (int32_t)C16);
+    reinterpret_cast<uint2 *>(P16)[i] = make_uint2(a | (b << 16), c | (d << 16));
+    reinterpret_cast<uint4 *>(Pd)[i] = make_uint4(a * 0x10001u, b * 0x10001u, c * 0x10001u, d * 0x10001u);
+  }
+}
+
+// k_check16 over a rank's owned UPPER tiles (the authoritative ones; D is symmetric, so the ranks
+// together cover every pair): a capped entry of a connected pair sets *flag = -1 (MIN-reducible)
+__global__ void k_check16_list(const uint16_t *__restrict__ S16, int64_t ld16, const int32_t *__restrict__ orow,
+                               int32_t nown, int32_t Np, const int32_t *__restrict__ lab, int32_t n_real,
+                               int32_t *flag) {
+  const int64_t per = (int64_t)TILE * (Np / 8);
+  const int64_t total = (int64_t)nown * per;
+  int found = 0;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
+    const int32_t lr = (int32_t)(i / per);
+    const int64_t rem = i % per;
+    const int32_t rr = (int32_t)(rem / (Np / 8)), c8 = (int32_t)(rem % (Np / 8)) * 8;
+    const int32_t r = orow[lr] * TILE + rr;
+    if (r >= n_real || c8 >= n_real || c8 < orow[lr] * TILE) continue;
+    const uint4 v = *reinterpret_cast<const uint4 *>(S16 + ((int64_t)lr * TILE + rr) * ld16 + c8);
+    const uint32_t w[4] = {v.x, v.y, v.z, v.w};
+#pragma unroll
+    for (int q = 0; q < 8; ++q) {
+      const uint32_t x = (w[q >> 1] >> ((q & 1) * 16)) & 0xFFFFu;
+      const int32_t c = c8 + q;
+      if (x == C16 && c < n_real && (!lab || lab[r] == lab[c])) found = 1;
+    }
+  }
+  if (__syncthreads_or(found) && threadIdx.x == 0) atomicMin(flag, -1);
+}
+
 // closure of the 16-bit pivot tile (ld Np), computed in int32 registers (values <= C16, so sums fit)
 __global__ void __launch_bounds__(NT, 1) k_fw_phase1_16(uint16_t *T, int64_t ldt) {
   __shared__ __align__(16) int32_t rowbuf[2][TILE];
@@ -515,9 +617,13 @@ struct TileJob16 {
   int64_t ldc;
   int32_t a_row0;    // row of the pivot row block inside tmA
   int32_t k, nt;
-  int32_t mode;      // MODE_PIVOT_ROW or MODE_UPPER
+  int32_t mode;      // MODE_PIVOT_ROW, MODE_UPPER, MODE_CROSS, MODE_REST or MODE_LIST
   int32_t mirror;
   int64_t ntiles;
+  // MODE_LIST (row-block sharded): as TileJob -- C holds the rank's owned tile rows only
+  const int32_t *orow;
+  const int64_t *opre;
+  int32_t nown, mk, posk;
 };
 
 template <int KC, int STAGES, int MINB, int UNR, int NTH = 256, int PFC = 0>
@@ -530,10 +636,10 @@ struct Fw16Cfg {
   static constexpr int RPH = 256 * 2 / NTH;   // row pairs per 64-row half owned by a thread (2 or 4)
 };
 
-__device__ __forceinline__ void decode16(const TileJob16 &J, int64_t idx, int &ti, int &tj) {
+__device__ __forceinline__ void decode16(const TileJob16 &J, int64_t idx, int &ti, int &tj, int &lr) {
   TileJob T{};
   T.k = J.k; T.nt = J.nt; T.mode = J.mode; T.ti0 = 0;
-  int lr;
+  T.orow = J.orow; T.opre = J.opre; T.nown = J.nown; T.mk = J.mk; T.posk = J.posk;
   decode_tile(T, idx, ti, tj, lr);
 }
 
@@ -555,13 +661,13 @@ __global__ void __launch_bounds__(CF::kNTH, CF::kMINB)
   const int my_tiles = J.ntiles > (int64_t)blockIdx.x ? (int)((J.ntiles - 1 - blockIdx.x) / gridDim.x + 1) : 0;
   const int total_chunks = my_tiles * NCHUNK;
   int issued = 0;
-  auto tile_of = [&](int it, int &ti, int &tj) { decode16(J, blockIdx.x + (int64_t)it * gridDim.x, ti, tj); };
+  auto tile_of = [&](int it, int &ti, int &tj, int &lr) { decode16(J, blockIdx.x + (int64_t)it * gridDim.x, ti, tj, lr); };
   auto produce = [&](int upto) {
     while (issued < upto) {
       const int st = issued % STAGES;
       if (issued >= STAGES) mbar_wait(&empty[st], (uint32_t)((issued / STAGES - 1) & 1));
-      int pti, ptj;
-      tile_of(issued / NCHUNK, pti, ptj);
+      int pti, ptj, plr;
+      tile_of(issued / NCHUNK, pti, ptj, plr);
       const int kc = issued % NCHUNK;
       mbar_arrive_tx(&full[st], CF::A_CHUNK * 2 + CF::B_CHUNK * 4);
       tma_load_2d(sA + st * CF::A_CHUNK, &tmA, pti * TILE, J.a_row0 + kc * KC, &full[st]);
@@ -584,10 +690,10 @@ __global__ void __launch_bounds__(CF::kNTH, CF::kMINB)
   auto row_of = [&](int r2) { return (r2 < RPH ? 0 : 64) + ty * 2 * RPH + (r2 % RPH) * 2; };
   int g = 0;
   for (int it = 0; it < my_tiles; ++it) {
-    int ti, tj;
-    tile_of(it, ti, tj);
+    int ti, tj, lr;
+    tile_of(it, ti, tj, lr);
     uint32_t c[NRP][8];
-    uint16_t *Ct = J.C + (int64_t)ti * TILE * J.ldc + (int64_t)tj * TILE;
+    uint16_t *Ct = J.C + (int64_t)lr * TILE * J.ldc + (int64_t)tj * TILE;
 #pragma unroll
     for (int r2 = 0; r2 < NRP; ++r2) {
       const int i = row_of(r2);
@@ -602,9 +708,9 @@ __global__ void __launch_bounds__(CF::kNTH, CF::kMINB)
       }
     }
     if (CF::kPFC && it + 1 < my_tiles) {   // pull the next tile's C rows into L2 while this one computes
-      int nti, ntj;
-      tile_of(it + 1, nti, ntj);
-      const uint16_t *Cn = J.C + (int64_t)nti * TILE * J.ldc + (int64_t)ntj * TILE;
+      int nti, ntj, nlr;
+      tile_of(it + 1, nti, ntj, nlr);
+      const uint16_t *Cn = J.C + (int64_t)nlr * TILE * J.ldc + (int64_t)ntj * TILE;
       // 128 rows x 256 B: one 128-byte line per (row, half), spread over the CTA's threads
       for (int l = tid; l < 2 * TILE; l += NTH)
         asm volatile("prefetch.global.L2::evict_last [%0];" ::"l"(Cn + (int64_t)(l >> 1) * J.ldc + (l & 1) * 64));
@@ -1104,6 +1210,149 @@ ear_status_t fw_sharded(int32_t *S, int64_t ldd, int32_t Np, ear_comm_s *comm, c
   return EAR_OK;
 }
 
+// ---------------------------------------------------------------- 16-bit row-block sharding
+// The sharded schedule above on packed 16-bit owned rows (the cap C16 and its exactness argument are
+// those of fw_single16).  The exchange stays int32 -- NCCL has no 16-bit MIN: the owned u16 pieces are
+// widened into the INF-filled int32 pivot row block, all-reduced, closed by the int32 phases 1-2 (on
+// capped inputs; min(x, C16) of their result is still exact, as the cap commutes with every
+// relaxation), then narrowed into the u16 A operand (also scattered back to the owners) and the
+// duplicated u32 B operand of the packed phase-3 kernel, which updates the owned u16 rows (MODE_LIST).
+// comm == nullptr: the shards are virtual ranks on this device sharing the block (their pieces are
+// disjoint, so no exchange is needed).  The range check runs over every rank's owned upper tiles and
+// is MIN-reduced; *done = false leaves the int32 owned storage untouched for the int32 schedule.
+static ear_status_t phase3_16(const Shard &sh, uint16_t *S16, const CUtensorMap &mA, const CUtensorMap &mB, int k,
+                              cudaStream_t st) {
+  int mk = 0, posk = -1;
+  int64_t total = 0;
+  for (int32_t r = 0; r < sh.nown; ++r) {
+    const int32_t ti = sh.rows[r];
+    if (ti < k) ++mk;
+    if (ti == k) posk = r;
+    total += ti == k ? 0 : (sh.nt - ti) - (ti < k ? 1 : 0);
+  }
+  TileJob16 J{S16, sh.Np, 0, k, sh.nt, MODE_LIST, 0, 0, sh.d_rows, sh.d_pre, sh.nown, mk, posk};
+  int s3 = prof_begin(PK_FW_P3_16, st);
+  EAR_TRY(launch16<Fw16Tile>(mA, mB, J, total, st));
+  prof_end(s3, st, (double)total * TILE * TILE * TILE);
+  return EAR_OK;
+}
+
+static ear_status_t fw_sharded16(std::vector<Shard *> &sh, int32_t Np, ear_comm_s *comm, const int32_t *lab,
+                                 int32_t n_real, bool *done, cudaStream_t st) {
+  *done = false;
+  const int nt = Np / TILE;
+  if (nt < 2) return EAR_OK;
+  if (!g_num_sms) {
+    int dev = 0;
+    EAR_CUDA_TRY(cudaGetDevice(&dev));
+    EAR_CUDA_TRY(cudaDeviceGetAttribute(&g_num_sms, cudaDevAttrMultiProcessorCount, dev));
+  }
+  const size_t R = sh.size();
+  std::vector<uint16_t *> S16(R, nullptr);
+  int32_t *prow = nullptr, *flag = nullptr;
+  uint16_t *p16 = nullptr;
+  uint32_t *Pd = nullptr;
+  bool ok = cudaMallocAsync((void **)&prow, sizeof(int32_t) * (size_t)TILE * Np, st) == cudaSuccess &&
+            cudaMallocAsync((void **)&p16, sizeof(uint16_t) * (size_t)TILE * Np, st) == cudaSuccess &&
+            cudaMallocAsync((void **)&Pd, sizeof(uint32_t) * (size_t)TILE * Np, st) == cudaSuccess &&
+            cudaMallocAsync((void **)&flag, sizeof(int32_t), st) == cudaSuccess;
+  for (size_t r = 0; r < R && ok; ++r)
+    ok = cudaMallocAsync((void **)&S16[r], sizeof(uint16_t) * (size_t)std::max(sh[r]->nown, 1) * TILE * Np, st) ==
+         cudaSuccess;
+  auto release = [&]() {
+    for (size_t r = 0; r < R; ++r)
+      if (S16[r]) cudaFreeAsync(S16[r], st);
+    if (prow) cudaFreeAsync(prow, st);
+    if (p16) cudaFreeAsync(p16, st);
+    if (Pd) cudaFreeAsync(Pd, st);
+    if (flag) cudaFreeAsync(flag, st);
+  };
+  if (!ok) {   // no room for the 16-bit copies: the int32 schedule runs
+    cudaGetLastError();
+    release();
+    return EAR_OK;
+  }
+  constexpr int KC = Fw16Tile::kKC;
+  const int64_t nblk = (int64_t)TILE * Np;
+  CUtensorMap map_prow, mA, mB;
+  ear_status_t s = make_map(&map_prow, prow, TILE, Np, Np, fw_kc());
+  if (s == EAR_OK) s = make_map_t(&mA, CU_TENSOR_MAP_DATA_TYPE_UINT16, 2, p16, TILE, Np, Np, KC);
+  if (s == EAR_OK) s = make_map_t(&mB, CU_TENSOR_MAP_DATA_TYPE_UINT32, 4, Pd, TILE, Np, Np, KC);
+  if (s == EAR_OK) {
+    int sc = prof_begin(PK_FW16_CONV, st);
+    for (size_t r = 0; r < R; ++r)
+      if (sh[r]->nown > 0)
+        EAR_LAUNCH(k_to16r, grid_for((int64_t)sh[r]->nown * TILE * (Np / 4)), 256, 0, st)(
+            sh[r]->S, sh[r]->ldd, S16[r], Np, (int64_t)sh[r]->nown * TILE, Np);
+    prof_end(sc, st, 0);
+  }
+  for (int k = 0; k < nt && s == EAR_OK; ++k) {
+    s = fill(prow, nblk, INF, st);
+    for (size_t r = 0; r < R && s == EAR_OK; ++r)
+      if (sh[r]->nown > 0)
+        EAR_LAUNCH(k_prow_xfer16<int32_t>, dim3(16, nt, sh[r]->nown), 256, 0, st)(S16[r], Np, sh[r]->d_rows, k, prow,
+                                                                                  Np, 0);
+    if (s == EAR_OK && comm) {
+      int sc = prof_begin(PK_COMM, st);
+      s = comm_allreduce_min(comm, prow, nblk, st);
+      prof_end(sc, st, 0);
+    }
+    if (s == EAR_OK) s = shard_pivot(prow, map_prow, Np, k, st);
+    if (s != EAR_OK) break;
+    EAR_LAUNCH(k_prow_to16, grid_for(nblk / 4), 256, 0, st)(prow, p16, Pd, nblk);
+    for (size_t r = 0; r < R; ++r)
+      if (sh[r]->nown > 0)
+        EAR_LAUNCH(k_prow_xfer16<uint16_t>, dim3(16, nt, sh[r]->nown), 256, 0, st)(S16[r], Np, sh[r]->d_rows, k, p16,
+                                                                                   Np, 1);
+    for (size_t r = 0; r < R && s == EAR_OK; ++r) s = phase3_16(*sh[r], S16[r], mA, mB, k, st);
+  }
+  int32_t h_flag = -1;
+  if (s == EAR_OK) {
+    int sc = prof_begin(PK_FW16_CONV, st);
+    cudaMemsetAsync(flag, 0, sizeof(int32_t), st);
+    for (size_t r = 0; r < R; ++r)
+      if (sh[r]->nown > 0)
+        EAR_LAUNCH(k_check16_list, grid_for((int64_t)sh[r]->nown * TILE * (Np / 8)), 256, 0, st)(
+            S16[r], Np, sh[r]->d_rows, sh[r]->nown, Np, lab, n_real, flag);
+    prof_end(sc, st, 0);
+    if (comm) s = comm_allreduce_min(comm, flag, 1, st);
+    cudaError_t e = cudaMemcpyAsync(&h_flag, flag, sizeof(int32_t), cudaMemcpyDeviceToHost, st);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+    if (s == EAR_OK && e != cudaSuccess) { set_error("fw_sharded16: %s", cudaGetErrorString(e)); s = EAR_ECUDA; }
+  }
+  if (s == EAR_OK && h_flag == 0) {
+    int sc = prof_begin(PK_FW16_CONV, st);
+    for (size_t r = 0; r < R; ++r)
+      if (sh[r]->nown > 0)
+        EAR_LAUNCH(k_from16r, grid_for((int64_t)sh[r]->nown * TILE * (Np / 4)), 256, 0, st)(
+            S16[r], Np, sh[r]->S, sh[r]->ldd, (int64_t)sh[r]->nown * TILE, Np);
+    prof_end(sc, st, 0);
+    *done = true;
+  }
+  release();
+  if (s != EAR_OK) return s;
+  EAR_CUDA_TRY(cudaGetLastError());
+  return EAR_OK;
+}
+
+// Sharded FW on a rank's owned int32 rows: the 16-bit schedule first (allow16), the int32 one when it
+// did not apply.  lab / n_real as for fw_single.
+ear_status_t fw_sharded_auto(int32_t *S, int64_t ldd, int32_t Np, ear_comm_s *comm, const int32_t *lab,
+                             int32_t n_real, bool allow16, cudaStream_t st) {
+  if (allow16 && Np >= 2 * TILE) {
+    Shard sh;
+    EAR_TRY(shard_setup(&sh, S, ldd, Np, comm->nranks, comm->rank, st));
+    std::vector<Shard *> v{&sh};
+    bool done = false;
+    ear_status_t s = fw_sharded16(v, Np, comm, lab, n_real, &done, st);
+    shard_free(&sh, st);
+    EAR_TRY(s);
+    prof_fw16(done);
+    if (done) return EAR_OK;
+  }
+  return fw_sharded(S, ldd, Np, comm, st);
+}
+
 // Full D from every rank's owned upper tiles (INF fill + scatter + all-reduce MIN).
 ear_status_t fw_sharded_gather(const int32_t *S, int64_t ldd, int32_t Np, int32_t *Df, int64_t ldf, ear_comm_s *comm,
                                cudaStream_t st) {
@@ -1150,7 +1399,7 @@ ear_status_t shard_rows_device(int32_t nt, int32_t P, int32_t rank, int32_t **d_
 // The same schedule for P ranks emulated in one process on one device (tests of the multi-GPU path on
 // one GPU): every virtual rank has its own owned storage, the shared prow stands in for the
 // all-reduce (the ranks' pieces are disjoint), and the ranks' upper tiles are scattered into D.
-ear_status_t fw_sharded_emulated(const ear_plan_s *plan, int32_t *D, int64_t ldd, int32_t Np, int32_t P,
+ear_status_t fw_sharded_emulated(ear_plan_s *plan, int32_t *D, int64_t ldd, int32_t Np, int32_t P,
                                  cudaStream_t st) {
   const int nt = Np / TILE;
   std::vector<Shard> sh(P);
@@ -1163,14 +1412,23 @@ ear_status_t fw_sharded_emulated(const ear_plan_s *plan, int32_t *D, int64_t ldd
     for (int32_t lr = 0; lr < sh[r].nown && status == EAR_OK; ++lr)
       status = fw_init_D(plan, S + (int64_t)lr * TILE * Np, Np, Np, sh[r].rows[lr] * TILE, TILE, st);
   }
+  bool done16 = false;
+  if (status == EAR_OK && !(plan->flags & EAR_FLAG_FW32) && Np >= 2 * TILE) {
+    const int32_t *lab = nullptr;
+    status = reduced_labels(plan, Np, st, &lab);
+    std::vector<Shard *> v;
+    for (int r = 0; r < P; ++r) v.push_back(&sh[r]);
+    if (status == EAR_OK) status = fw_sharded16(v, Np, nullptr, lab, plan->n_reduced, &done16, st);
+    if (status == EAR_OK) prof_fw16(done16);
+  }
   int32_t *prow = nullptr;
-  if (status == EAR_OK) {
+  if (status == EAR_OK && !done16) {
     cudaError_t e = cudaMallocAsync((void **)&prow, sizeof(int32_t) * (size_t)TILE * Np, st);
     if (e != cudaSuccess) { set_error("emulated prow: %s", cudaGetErrorString(e)); status = EAR_ENOMEM; }
   }
   CUtensorMap map_prow;
-  if (status == EAR_OK) status = make_map(&map_prow, prow, TILE, Np, Np, fw_kc());
-  for (int k = 0; k < nt && status == EAR_OK; ++k) {
+  if (status == EAR_OK && !done16) status = make_map(&map_prow, prow, TILE, Np, Np, fw_kc());
+  for (int k = 0; k < nt && status == EAR_OK && !done16; ++k) {
     status = fill(prow, (int64_t)TILE * Np, INF, st);
     for (int r = 0; r < P && status == EAR_OK; ++r) status = shard_xfer(sh[r], k, prow, 0, st);
     if (status == EAR_OK) status = shard_pivot(prow, map_prow, Np, k, st);

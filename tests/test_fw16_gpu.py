@@ -139,3 +139,65 @@ def test_bcc_pieces_16bit(pkg, seed):
     ref = oracle_on_terminals(g)
     got, prof = reduced(pkg, g, flags=pkg.FLAG_BCC)
     assert_exact(got, ref, f"bcc corner seed {seed}")
+
+
+# ------------------------------------------------------------- the 16-bit row-block sharded schedule
+def emulated(pkg, g, P, flags=0):
+    """D on V^r from the P-rank sharded schedule emulated on this GPU, with its profile."""
+    plan = pkg.ear_decompose(g.n, dev(g.src), dev(g.dst), dev(g.w), flags=flags)
+    pkg.profile_reset()
+    pkg.profile_enable(True)
+    D = pkg.apsp_reduced_emulated(plan, P)
+    torch.cuda.synchronize()
+    prof = pkg.profile_read()
+    pkg.profile_enable(False)
+    nr = plan.info().n_reduced
+    out = D[:nr, :nr].cpu().numpy()
+    plan.destroy()
+    return out, prof
+
+
+@pytest.mark.parametrize("P", [1, 2, 3, 4, 8])
+def test_sharded16_kept(pkg, P):
+    """Every virtual rank runs the packed kernel on its owned rows (MODE_LIST) and the result is kept."""
+    g = gg.config("cfg1")
+    got, prof = emulated(pkg, g, P)
+    assert prof["fw16_used"] == 1 and prof["fw16_fallbacks"] == 0 and prof["fw_phase3_16_minplus"] > 0
+    assert_exact(got, oracle_on_terminals(g), f"sharded16 P={P}")
+
+
+@pytest.mark.parametrize("P", [2, 5])
+def test_sharded16_fallback(pkg, P):
+    g = ladder(700, 100, seed=7)
+    got, prof = emulated(pkg, g, P)
+    assert prof["fw16_used"] == 0 and prof["fw16_fallbacks"] == 1
+    assert_exact(got, oracle_on_terminals(g), f"sharded16 fallback P={P}")
+
+
+@pytest.mark.parametrize("delta", [-1, 0])
+def test_sharded16_cap_boundary(pkg, delta):
+    L, a = 300, 100
+    target = CAP - 1 if delta == -1 else CAP
+    g = ladder(L, a, rung_w=target - (L - 3) * a)
+    got, prof = emulated(pkg, g, 3)
+    assert prof["fw16_used"] == (1 if delta == -1 else 0)
+    assert_exact(got, oracle_on_terminals(g), f"sharded16 boundary {target}")
+
+
+def test_sharded16_disconnected(pkg):
+    a, b = ladder(200, 30, seed=8), ladder(150, 40, seed=9)
+    g = gg.Graph(a.n + b.n, np.concatenate([a.src, b.src + a.n]).astype(np.int32),
+                 np.concatenate([a.dst, b.dst + a.n]).astype(np.int32), np.concatenate([a.w, b.w]).astype(np.int32))
+    got, prof = emulated(pkg, g, 4)
+    assert prof["fw16_used"] == 1
+    assert_exact(got, oracle_on_terminals(g), "sharded16 two components")
+
+
+@pytest.mark.parametrize("seed", range(3))
+def test_sharded16_corner_equals_fw32(pkg, seed):
+    g = gg.corner_cases(4100 + seed, n_target=900 + 300 * seed)
+    d16, p16 = emulated(pkg, g, 3)
+    d32, p32 = emulated(pkg, g, 3, flags=pkg.FLAG_FW32)
+    assert p32["fw16_used"] == 0 and p32["fw16_fallbacks"] == 0
+    assert np.array_equal(d16, d32)
+    assert_exact(d16, oracle_on_terminals(g), f"sharded16 corner seed {seed}")

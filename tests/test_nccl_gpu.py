@@ -1,7 +1,8 @@
 """The NCCL path on one GPU: a communicator of ONE rank (torch.distributed nccl process group, NCCL
 unique id from the library) runs the sharded schedule with its real ncclAllReduce(MIN) of the pivot
 row block every FW round and of the final D (and the sharded SSSP Phase II), then the expansion --
-bit-exact against the oracle.  (The multi-rank schedule
+bit-exact against the oracle; with the default flags the packed 16-bit sharded FW runs, FLAG_FW32 the
+int32 one, FLAG_BCC shards the largest biconnected piece.  (The multi-rank schedule
 itself is checked on one GPU by test_parity_gpu.py::test_sharded_schedule_emulated.)"""
 import os
 import socket
@@ -24,7 +25,7 @@ comm = ea.Comm.from_torch_distributed()
 dev = lambda a: torch.as_tensor(np.ascontiguousarray(a, dtype=np.int32)).cuda()
 for g in [gg.config("cfg1"), gg.corner_cases(12, n_target=500)]:
     ref = oracle.apsp(g.n, g.src, g.dst, g.w)
-    for flags in (0, ea.FLAG_SSSP):
+    for flags in (0, ea.FLAG_SSSP, ea.FLAG_BCC, ea.FLAG_FW32, ea.FLAG_BCC | ea.FLAG_FW32):
         out = ea.apsp_full(g.n, dev(g.src), dev(g.dst), dev(g.w), comm=comm, flags=flags)
         torch.cuda.synchronize()
         assert np.array_equal(out.cpu().numpy(), ref), f"nccl path mismatch (flags={flags})"

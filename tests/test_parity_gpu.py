@@ -237,13 +237,14 @@ def test_invalid_inputs_raise(pkg):
 
 
 # ------------------------------------------------------------------------------ multi-GPU schedule
+@pytest.mark.parametrize("fw32", [False, True])
 @pytest.mark.parametrize("P", [1, 2, 3, 4, 8])
-def test_sharded_schedule_emulated(pkg, P):
+def test_sharded_schedule_emulated(pkg, P, fw32):
     """P7: the row-block-sharded FW schedule (owner phase 1 + pivot-row tiles -> pivot broadcast ->
     per-rank pivot-column tiles by symmetry + phase 3) emulated for P ranks on this GPU equals the
     single-GPU symmetric FW bit for bit, and the oracle on V^r."""
     g = gg.config("cfg1")
-    plan = pkg.ear_decompose(g.n, dev(g.src), dev(g.dst), dev(g.w))
+    plan = pkg.ear_decompose(g.n, dev(g.src), dev(g.dst), dev(g.w), flags=pkg.FLAG_FW32 if fw32 else 0)
     nr = plan.info().n_reduced
     D1 = pkg.alloc_D(plan)
     pkg.apsp_reduced(plan, D1)
