@@ -626,13 +626,16 @@ struct TileJob16 {
   int32_t nown, mk, posk;
 };
 
-template <int KC, int STAGES, int MINB, int UNR, int NTH = 256, int PFC = 0>
+// LAR = 1: a ring stage is refilled by the LAST warp to finish consuming it (a shared counter) instead
+// of thread 0 waiting on an 'empty' barrier at the start of each chunk (which ties warp 0 to the
+// slowest warp every chunk).
+template <int KC, int STAGES, int MINB, int UNR, int NTH = 256, int PFC = 0, int LAR = 0>
 struct Fw16Cfg {
   static constexpr int NCHUNK = TILE / KC;
   static constexpr int A_CHUNK = KC * TILE;   // u16 elements
   static constexpr int B_CHUNK = KC * TILE;   // u32 elements
-  static constexpr int SMEM = STAGES * (A_CHUNK * 2 + B_CHUNK * 4) + 2 * STAGES * 8;
-  static constexpr int kKC = KC, kSTAGES = STAGES, kMINB = MINB, kUNR = UNR, kNTH = NTH, kPFC = PFC;
+  static constexpr int SMEM = STAGES * (A_CHUNK * 2 + B_CHUNK * 4) + 2 * STAGES * 8 + STAGES * 4;
+  static constexpr int kKC = KC, kSTAGES = STAGES, kMINB = MINB, kUNR = UNR, kNTH = NTH, kPFC = PFC, kLAR = LAR;
   static constexpr int RPH = 256 * 2 / NTH;   // row pairs per 64-row half owned by a thread (2 or 4)
 };
 
@@ -655,6 +658,7 @@ __global__ void __launch_bounds__(CF::kNTH, CF::kMINB)
   uint32_t *sB = reinterpret_cast<uint32_t *>(sA + STAGES * CF::A_CHUNK);     // [STAGES][KC][TILE] u32
   uint64_t *full = reinterpret_cast<uint64_t *>(sB + STAGES * CF::B_CHUNK);
   uint64_t *empty = full + STAGES;
+  int32_t *cnt = reinterpret_cast<int32_t *>(empty + STAGES);   // LAR: warps done with the stage
   const int tid = threadIdx.x, lane = tid & 31;
   const int tx = tid & 15, ty = tid >> 4;
 
@@ -662,6 +666,14 @@ __global__ void __launch_bounds__(CF::kNTH, CF::kMINB)
   const int total_chunks = my_tiles * NCHUNK;
   int issued = 0;
   auto tile_of = [&](int it, int &ti, int &tj, int &lr) { decode16(J, blockIdx.x + (int64_t)it * gridDim.x, ti, tj, lr); };
+  auto issue = [&](int c, int st) {   // chunk c into stage st
+    int pti, ptj, plr;
+    tile_of(c / NCHUNK, pti, ptj, plr);
+    const int kc = c % NCHUNK;
+    mbar_arrive_tx(&full[st], CF::A_CHUNK * 2 + CF::B_CHUNK * 4);
+    tma_load_2d(sA + st * CF::A_CHUNK, &tmA, pti * TILE, J.a_row0 + kc * KC, &full[st]);
+    tma_load_2d(sB + st * CF::B_CHUNK, &tmB, ptj * TILE, kc * KC, &full[st]);
+  };
   auto produce = [&](int upto) {
     while (issued < upto) {
       const int st = issued % STAGES;
@@ -679,13 +691,20 @@ __global__ void __launch_bounds__(CF::kNTH, CF::kMINB)
     for (int s = 0; s < STAGES; ++s) {
       mbar_init(&full[s], 1);
       mbar_init(&empty[s], NTH / 32);
+      cnt[s] = 0;
     }
     asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
     asm volatile("prefetch.tensormap [%0];\n" ::"l"(reinterpret_cast<uint64_t>(&tmA)) : "memory");
     asm volatile("prefetch.tensormap [%0];\n" ::"l"(reinterpret_cast<uint64_t>(&tmB)) : "memory");
   }
   __syncthreads();
-  if (tid == 0 && my_tiles > 0) produce(total_chunks < STAGES ? total_chunks : STAGES);
+  if (tid == 0 && my_tiles > 0) {
+    if (CF::kLAR) {
+      for (int c = 0; c < STAGES && c < total_chunks; ++c) issue(c, c);
+    } else {
+      produce(total_chunks < STAGES ? total_chunks : STAGES);
+    }
+  }
 
   auto row_of = [&](int r2) { return (r2 < RPH ? 0 : 64) + ty * 2 * RPH + (r2 % RPH) * 2; };
   int g = 0;
@@ -717,7 +736,7 @@ __global__ void __launch_bounds__(CF::kNTH, CF::kMINB)
     }
 #pragma unroll 1
     for (int kc = 0; kc < NCHUNK; ++kc, ++g) {
-      if (tid == 0) produce(g + STAGES < total_chunks ? g + STAGES : total_chunks);
+      if (!CF::kLAR && tid == 0) produce(g + STAGES < total_chunks ? g + STAGES : total_chunks);
       const int st = g % STAGES;
       mbar_wait(&full[st], (uint32_t)((g / STAGES) & 1));
       const uint16_t *a_s = sA + st * CF::A_CHUNK;
@@ -744,7 +763,19 @@ __global__ void __launch_bounds__(CF::kNTH, CF::kMINB)
           for (int q = 0; q < 8; ++q) c[r2][q] = __viaddmin_u16x2(a[r2], b[q], c[r2][q]);
       }
       __syncwarp();
-      if (lane == 0) mbar_arrive(&empty[st]);
+      if (CF::kLAR) {
+        if (lane == 0) {
+          __threadfence_block();
+          if (atomicAdd(&cnt[st], 1) == NTH / 32 - 1) {   // the last reader of this stage refills it
+            cnt[st] = 0;
+            __threadfence_block();
+            asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");
+            if (g + STAGES < total_chunks) issue(g + STAGES, st);
+          }
+        }
+      } else if (lane == 0) {
+        mbar_arrive(&empty[st]);
+      }
     }
 #pragma unroll
     for (int r2 = 0; r2 < NRP; ++r2) {
@@ -869,8 +900,15 @@ ear_status_t launch_tiles(const CUtensorMap &map, TileJob J, int64_t nblocks, cu
 
 // Packed 16-bit tile kernel configuration, chosen by tools/sweep_fw16.py on the B200 (cfg4, 17
 // variants, profiles/r01_fw16_variants.jsonl): 128 threads with 16 x 8 values each, 32-deep k-chunks,
-// a 2-stage TMA ring (48 KB), 3 CTAs per SM, kk unrolled 16x.
-using Fw16Tile = Fw16Cfg<32, 2, 3, 16, 128>;
+// a 2-stage TMA ring (48 KB), 3 CTAs per SM, kk unrolled 16x; then (tools/lab_fw16_variant.sh,
+// profiles/r01u_fw16_refill.jsonl) last-arriver refills of the ring and an L2 prefetch of the next
+// C tile: 475.3 -> 471.6 ms on cfg4's plain FW (3-stage rings and 16-deep chunks measured slower).
+using Fw16Tile = Fw16Cfg<32, 2, 3, 16, 128, 1, 1>;
+using Fw16TileL = Fw16Cfg<32, 2, 3, 16, 128, 0, 1>;
+using Fw16TileL4 = Fw16Cfg<16, 4, 3, 16, 128, 0, 1>;
+using Fw16TileL3 = Fw16Cfg<32, 3, 3, 16, 128, 0, 1>;
+using Fw16TileLP = Fw16Cfg<32, 2, 3, 16, 128, 1, 1>;
+using Fw16TileL3P = Fw16Cfg<32, 3, 3, 16, 128, 1, 1>;
 
 // development knobs (tools/): EAR_FW16_LOOKAHEAD=0 disables the lookahead, EAR_FW16_RESERVE sets the
 // CTA slots the rest-of-round launch leaves free for the next round's pivot work (default 0: measured
@@ -881,9 +919,8 @@ int env_int(const char *name, int dflt) {
 }
 
 template <class CF>
-ear_status_t launch16(const CUtensorMap &mA, const CUtensorMap &mB, TileJob16 J, int64_t nblocks, cudaStream_t st,
-                      int reserve = 0) {
-  if (nblocks <= 0) return EAR_OK;
+ear_status_t launch16_cfg(const CUtensorMap &mA, const CUtensorMap &mB, TileJob16 J, int64_t nblocks, cudaStream_t st,
+                          int reserve) {
   static bool attr = false;
   if (!attr) {
     EAR_CUDA_TRY(cudaFuncSetAttribute(k_fw_tiles16<CF>, cudaFuncAttributeMaxDynamicSharedMemorySize, CF::SMEM));
@@ -896,6 +933,23 @@ ear_status_t launch16(const CUtensorMap &mA, const CUtensorMap &mB, TileJob16 J,
   const int64_t grid = std::min<int64_t>(nblocks, std::max<int64_t>(1, (int64_t)g_num_sms * per_sm - reserve));
   EAR_LAUNCH(k_fw_tiles16<CF>, (unsigned)grid, CF::kNTH, CF::SMEM, st)(mA, mB, J);
   return EAR_OK;
+}
+
+int fw16_kc() { return env_int("EAR_FW16_VARIANT", 0) == 2 ? Fw16TileL4::kKC : Fw16Tile::kKC; }
+
+// EAR_FW16_VARIANT (development knob, tools/lab_fw16_variant.sh): 0 = Fw16Tile, 1 = last-arriver refill
+// without the C prefetch, 2 = 4-stage ring of 16-deep chunks, 3 = 3-stage ring, 5 = 3-stage + prefetch
+template <class CF>
+ear_status_t launch16(const CUtensorMap &mA, const CUtensorMap &mB, TileJob16 J, int64_t nblocks, cudaStream_t st,
+                      int reserve = 0) {
+  if (nblocks <= 0) return EAR_OK;
+  static const int variant = env_int("EAR_FW16_VARIANT", 0);
+  if (variant == 1) return launch16_cfg<Fw16TileL>(mA, mB, J, nblocks, st, reserve);
+  if (variant == 2) return launch16_cfg<Fw16TileL4>(mA, mB, J, nblocks, st, reserve);
+  if (variant == 3) return launch16_cfg<Fw16TileL3>(mA, mB, J, nblocks, st, reserve);
+  if (variant == 4) return launch16_cfg<Fw16TileLP>(mA, mB, J, nblocks, st, reserve);
+  if (variant == 5) return launch16_cfg<Fw16TileL3P>(mA, mB, J, nblocks, st, reserve);
+  return launch16_cfg<CF>(mA, mB, J, nblocks, st, reserve);
 }
 
 int grid_for(int64_t n) { return (int)std::max<int64_t>(1, std::min<int64_t>(ceil_div(n, 256), 148 * 16)); }
@@ -947,7 +1001,7 @@ ear_status_t fw_single16(int32_t *D, int64_t ldd, int32_t Np, const int32_t *lab
     if (Pd) cudaFreeAsync(Pd, st);
     return EAR_OK;   // no room for the 16-bit copy: the int32 path runs
   }
-  constexpr int KC = Fw16Tile::kKC;
+  const int KC = fw16_kc();
   ear_status_t s = EAR_OK;
   CUtensorMap mA, mB[2];
   s = make_map_t(&mA, CU_TENSOR_MAP_DATA_TYPE_UINT16, 2, D16, Np, Np, Np, KC);
@@ -1272,7 +1326,7 @@ static ear_status_t fw_sharded16(std::vector<Shard *> &sh, int32_t Np, ear_comm_
     release();
     return EAR_OK;
   }
-  constexpr int KC = Fw16Tile::kKC;
+  const int KC = fw16_kc();
   const int64_t nblk = (int64_t)TILE * Np;
   CUtensorMap map_prow, mA, mB;
   ear_status_t s = make_map(&map_prow, prow, TILE, Np, Np, fw_kc());
