@@ -167,6 +167,11 @@ typedef struct {
   int32_t largest_piece;  /* vertices of the largest piece */
   int32_t tree_levels;    /* levels of the BFS spanning forest (latency of the tree sweeps) */
   double sum_cubes;       /* sum over pieces of size^3 (FW work; N_r^3 without EAR_FLAG_BCC) */
+  int32_t rereduced_pieces;  /* big pieces that the last solve reduced again (each block is
+                                reduced; an articulation point can have degree 2 inside its block) */
+  int32_t largest_reduced;   /* size the largest piece's FW ran on in the last solve (0 before one) */
+  int32_t rereduce_levels;   /* most nested reductions of one piece in the last solve (a reduced
+                                piece is reduced again while that removes >= 1 % of its vertices) */
 } ear_bcc_info_t;
 ear_status_t ear_bcc_info(ear_plan_t plan, ear_bcc_info_t *info);
 

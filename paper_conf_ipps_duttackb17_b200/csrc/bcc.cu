@@ -48,6 +48,8 @@ struct ear_bcc_s {
   std::vector<int32_t> h_psize, h_pld;
   std::vector<int64_t> h_pbase;
   std::vector<int32_t> big;                   // pieces with more than 128 vertices (blocked FW)
+  int32_t rereduced = 0, largest_reduced = 0;  // last solve: big pieces reduced again, largest's size
+  int32_t rereduce_levels = 0;                 // most nested reductions applied to one piece
 };
 
 namespace ear {
@@ -403,6 +405,18 @@ __global__ void k_pool_init(int32_t nr, const int4 *cinfo, const int32_t *ridx, 
   }
 }
 
+// the arcs of piece `pc` as a piece-local edge list (both directions; decompose() merges them)
+__global__ void k_piece_edges(const int4 *arcs, int32_t A, int32_t pc, int32_t *u, int32_t *v, int32_t *w,
+                              int32_t *cnt) {
+  GS(a, A) {
+    const int4 e = arcs[a];
+    if (e.x == pc && e.y < e.z) {
+      const int32_t i = atomicAdd(cnt, 1);
+      u[i] = e.y; v[i] = e.z; w[i] = e.w;
+    }
+  }
+}
+
 // one CTA per piece of 3..128 vertices: plain Floyd-Warshall in shared memory (P:101 per block)
 __global__ void __launch_bounds__(NT) k_piece_fw(int32_t np, const int32_t *psize, const int32_t *pld,
                                                  const int64_t *pbase, int32_t *pool) {
@@ -668,6 +682,106 @@ ear_status_t fw_sharded_gather(const int32_t *S, int64_t ldd, int32_t Np, int32_
 std::vector<int32_t> shard_rows(int32_t nt, int32_t P, int32_t rank);
 int32_t shard_nown(int32_t nt, int32_t P, int32_t rank);
 
+// The paper's order inside a big piece (G is split into its biconnected components and EACH is
+// then reduced): a vertex of degree >= 3 in G^r can have degree 2 inside its block (an articulation
+// point with one edge to a hanging piece), so the piece is reduced again -- Phase I on the piece's
+// local edge list -- and the piece matrix M (ld, piece-local ids) is Phase III of that reduction over
+// the FW of the smaller reduced piece.  Used when the reduced piece needs fewer 128-tiles; *done =
+// false leaves M for the FW on the whole piece.  With a communicator the reduced
+// piece is row-block sharded and gathered, and every rank expands M (all ranks need the whole piece).
+constexpr int REREDUCE_DEPTH = 4;
+
+// Distance matrix M (n x n, ld) of a connected graph given as an edge list, by the paper's method
+// applied to it: Reduce (Phase I) -> distances of the reduced graph -> UPDATE_DISTANCE (Phase III).
+// The reduced graph's distances come from the same recursion when its own Reduce still saves a tile
+// (merging parallel edges can leave new degree-two vertices), else
+// from the FW (sharded with a communicator).  *done = false (nothing written) when Reduce saves no
+// tile at the top level.  *levels / *n_last: reductions applied and the size the FW ran on.
+static ear_status_t reduce_solve(const ear_plan_s *p, int32_t n, int64_t m, const int32_t *u, const int32_t *v,
+                                 const int32_t *w, int32_t *M, int64_t ld, ear_comm_s *comm, int depth,
+                                 cudaStream_t st, bool *done, int32_t *levels, int32_t *n_last) {
+  *done = false;
+  ear_plan_s *q = new ear_plan_s;
+  q->device = p->device;
+  ear_status_t s = decompose(n, m, u, v, w, p->flags & EAR_FLAG_FW32, st, q);
+  // worth it when the FW runs on fewer 128-tiles (same tile count: same FW work, plus the expansion)
+  const int64_t unit = (int64_t)TILE * (comm ? comm->nranks : 1);
+  const bool worth = s == EAR_OK && round_up(std::max<int64_t>(q->n_reduced, 1), unit) < round_up(n, unit);
+  if (!worth) {
+    cudaStreamSynchronize(st);
+    plan_free(q);
+    delete q;
+    return s;
+  }
+  *levels = depth + 1;
+  *n_last = q->n_reduced;
+  const int32_t P = comm ? comm->nranks : 1;
+  const int32_t Np = (int32_t)round_up(std::max<int64_t>(q->n_reduced, 1), (int64_t)TILE * P);
+  const bool allow16 = !(p->flags & EAR_FLAG_FW32);
+  int32_t *D = nullptr;
+  bool inner = false;
+  if (cudaMallocAsync((void **)&D, sizeof(int32_t) * (size_t)Np * Np, st) != cudaSuccess) {
+    set_error("bcc_solve: out of device memory (re-reduced piece)");
+    s = EAR_ENOMEM;
+  }
+  if (s == EAR_OK && depth + 1 < REREDUCE_DEPTH && q->n_redges > 0)
+    s = reduce_solve(p, q->n_reduced, q->n_redges, q->re_u, q->re_v, q->re_w, D, Np, comm, depth + 1, st, &inner,
+                     levels, n_last);
+  if (s == EAR_OK && !inner) {
+    if (!comm) {
+      s = fw_init_D(q, D, Np, Np, 0, Np, st);
+      if (s == EAR_OK) s = fw_single(D, Np, Np, st, nullptr, q->n_reduced, allow16);   // connected
+    } else {
+      const std::vector<int32_t> own = shard_rows(Np / TILE, P, comm->rank);
+      int32_t *S = nullptr;
+      if (cudaMallocAsync((void **)&S, sizeof(int32_t) * std::max<size_t>(own.size(), 1) * TILE * Np, st) !=
+          cudaSuccess) {
+        set_error("bcc_solve: out of device memory (re-reduced piece)");
+        s = EAR_ENOMEM;
+      }
+      for (size_t j = 0; j < own.size() && s == EAR_OK; ++j)
+        s = fw_init_D(q, S + (int64_t)j * TILE * Np, Np, Np, own[j] * TILE, TILE, st);
+      if (s == EAR_OK) s = fw_sharded_auto(S, Np, Np, comm, nullptr, q->n_reduced, allow16, st);
+      if (s == EAR_OK) s = fw_sharded_gather(S, Np, Np, D, Np, comm, st);
+      if (S) cudaFreeAsync(S, st);
+    }
+  }
+  if (s == EAR_OK) s = expand(q, D, Np, 0, n, M, ld, st);
+  if (D) cudaFreeAsync(D, st);
+  cudaStreamSynchronize(st);   // q's arrays are freed below
+  plan_free(q);
+  delete q;
+  if (s == EAR_OK) *done = true;
+  return s;
+}
+
+// The paper's order inside a big piece: its local edge list -> reduce_solve.
+static ear_status_t piece_rereduce(ear_plan_s *p, ear_bcc_s *b, int32_t id, int32_t *M, int32_t ld, ear_comm_s *comm,
+                                   cudaStream_t st, bool *done, int32_t *n_reduced) {
+  *done = false;
+  if (getenv("EAR_NO_REREDUCE")) return EAR_OK;   // development knob (A/B timing)
+  const int32_t np = b->h_psize[id];
+  const int32_t A = b->n_arcs;
+  if (A <= 0) return EAR_OK;
+  int32_t *e = nullptr;
+  EAR_CUDA_TRY(cudaMallocAsync((void **)&e, sizeof(int32_t) * (3 * (size_t)A + 1), st));
+  int32_t *cnt = e + 3 * (size_t)A;
+  EAR_CUDA_TRY(cudaMemsetAsync(cnt, 0, sizeof(int32_t), st));
+  EAR_LAUNCH(k_piece_edges, grid_for(A), NT, 0, st)(b->arcs, A, id, e, e + A, e + 2 * (size_t)A, cnt);
+  int32_t m = 0;
+  EAR_CUDA_TRY(cudaMemcpyAsync(&m, cnt, sizeof(int32_t), cudaMemcpyDeviceToHost, st));
+  EAR_CUDA_TRY(cudaStreamSynchronize(st));
+  int32_t levels = 0, n_last = np;
+  ear_status_t s = reduce_solve(p, np, m, e, e + A, e + 2 * (size_t)A, M, ld, comm, 0, st, done, &levels, &n_last);
+  cudaFreeAsync(e, st);
+  if (s == EAR_OK && *done) {
+    *n_reduced = n_last;
+    b->rereduced++;
+    b->rereduce_levels = std::max(b->rereduce_levels, levels);
+  }
+  return s;
+}
+
 // Phase II by blocks: solve every piece, then compose rows of S^r into D.  Rows: [row0, row0 + rows)
 // or, with d_tile_rows, the listed 128-row blocks (comm layout).  With a communicator the largest
 // piece runs the sharded FW (its rows split over the ranks) and is re-assembled on every rank; the
@@ -693,10 +807,18 @@ ear_status_t bcc_solve(ear_plan_s *p, ear_comm_s *comm, int32_t *D, int64_t ldd,
   if (b->n_pieces > 0)
     EAR_LAUNCH(k_piece_fw, b->n_pieces, NT, SMALL * SMALL * 4, st)(b->n_pieces, b->psize, b->pld, b->pbase, pool);
   prof_end(sp, st, 0);
+  b->rereduced = 0;
+  b->rereduce_levels = 0;
+  b->largest_reduced = b->big.empty() ? b->largest : 0;
   for (size_t i = 0; i < b->big.size() && s == EAR_OK; ++i) {
     const int32_t id = b->big[i];
     int32_t *M = pool + b->h_pbase[id];
     const int32_t ld = b->h_pld[id];
+    bool done = false;
+    int32_t nred = b->h_psize[id];
+    s = piece_rereduce(p, b, id, M, ld, (comm && i == 0) ? comm : nullptr, st, &done, &nred);
+    if (i == 0) b->largest_reduced = nred;
+    if (s != EAR_OK || done) continue;
     if (comm && i == 0) {   // the largest piece: sharded over the ranks, then gathered everywhere
       const int32_t nt = ld / TILE;
       std::vector<int32_t> own = shard_rows(nt, P, comm->rank);
@@ -755,5 +877,8 @@ extern "C" ear_status_t ear_bcc_info(ear_plan_t p, ear_bcc_info_t *info) {
   info->largest_piece = b->largest;
   info->tree_levels = b->levels;
   info->sum_cubes = b->sum_cubes;
+  info->rereduced_pieces = b->rereduced;
+  info->largest_reduced = b->largest_reduced;
+  info->rereduce_levels = b->rereduce_levels;
   return EAR_OK;
 }

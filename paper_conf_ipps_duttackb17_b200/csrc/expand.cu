@@ -10,7 +10,8 @@
 //     same chain: S[s, t] = min(S[s, t], |off_s - off_t|)            P:107 (readings C8, C9)
 // then clamped to EAR_INF.
 //
-// k_expand: one CTA per group of RB = 32 consecutive output rows; its distinct chain ends E (<= 64)
+// k_expand: persistent CTAs take work items in order -- a group of RB = 32 consecutive output rows
+// (the last ~wave of groups split into column segments); a group's distinct chain ends E (<= 64)
 // are split greedily into sub-groups of <= ECAP endpoints.  Each of the 8 warps owns a 128-column
 // slice of every 1,024-column chunk and works independently of the others (no CTA barrier in the
 // main loop):
@@ -41,6 +42,9 @@ constexpr int RB = 32;              // rows per CTA
 constexpr int ECAP = 16;            // endpoints per sub-group (R tile: ECAP x 1024 ints = 64 KB)
 constexpr int CHUNK = 1024;         // columns per chunk (8 warps x 128)
 constexpr int BATCH = 4;            // ends per gather batch
+#ifndef EXP_MINB
+#define EXP_MINB 2
+#endif
 constexpr int EXP_SMEM = ECAP * CHUNK * 4;
 
 __device__ __forceinline__ void st_cs_v4(int32_t *p, int4 v) {
@@ -62,9 +66,19 @@ __device__ __forceinline__ int32_t *row_ptr(int32_t *base, int32_t r, uint32_t l
   return reinterpret_cast<int32_t *>(reinterpret_cast<char *>(base) + (uint64_t)(uint32_t)r * ld_bytes);
 }
 
-__global__ void __launch_bounds__(NT, 2) k_expand(const int32_t *__restrict__ D, int64_t ldd,
+// Work items, taken in order from a global counter by persistent CTAs (one wave): items [0, n_full)
+// are whole row groups (all n columns); the last row groups -- about one wave of them -- are split
+// into nseg column segments of seg_w columns (a multiple of CHUNK), so the launch ends with small
+// items instead of a partial wave of whole row groups.
+struct ExpandWork {
+  int32_t *counter;
+  int32_t n_full, n_items, nseg, seg_w;
+};
+
+__global__ void __launch_bounds__(NT, EXP_MINB) k_expand(const int32_t *__restrict__ D, int64_t ldd,
                                                  const VDesc *__restrict__ desc, int32_t n, int32_t row_begin,
-                                                 int32_t row_end, int32_t *__restrict__ out, int64_t ldo) {
+                                                 int32_t row_end, int32_t *__restrict__ out, int64_t ldo,
+                                                 const ExpandWork W) {
   extern __shared__ __align__(16) int32_t R[];       // [ECAP][CHUNK]
   __shared__ VDesc rdesc[RB];
   __shared__ int32_t ends[2 * RB];                   // endpoint tids, sub-group by sub-group
@@ -74,10 +88,21 @@ __global__ void __launch_bounds__(NT, 2) k_expand(const int32_t *__restrict__ D,
   __shared__ int8_t sg_row0[RB + 1], sg_e0[RB + 1];  // sub-group g: rows [row0[g], row0[g+1]), ends [e0[g], e0[g+1])
   __shared__ int4 meta[RB];                          // chain rows by sub-group: {cp, cq, ip | iq << 8, local row}
   __shared__ int8_t sg_m0[RB + 1];
-  __shared__ int32_t n_sg;
+  __shared__ int32_t n_sg, item_sh;
 
   const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
-  const int32_t r0 = row_begin + blockIdx.x * RB;
+  for (;;) {
+  if (tid == 0) item_sh = atomicAdd(W.counter, 1);
+  __syncthreads();
+  const int32_t item = item_sh;
+  if (item >= W.n_items) break;
+  int32_t rg = item, col_b = 0, col_e = n;
+  if (item >= W.n_full) {
+    rg = W.n_full + (item - W.n_full) / W.nseg;
+    col_b = ((item - W.n_full) % W.nseg) * W.seg_w;
+    col_e = min(n, col_b + W.seg_w);
+  }
+  const int32_t r0 = row_begin + rg * RB;
   const int nrows = min(RB, row_end - r0);
   if (tid < nrows) rdesc[tid] = desc[r0 + tid];
   __syncthreads();
@@ -131,7 +156,7 @@ __global__ void __launch_bounds__(NT, 2) k_expand(const int32_t *__restrict__ D,
   const uint32_t ldo_b = (uint32_t)(ldo * 4);
   int32_t *const oblk = out + (int64_t)(r0 - row_begin) * ldo;   // this CTA's first output row
   int32_t *Rw = R + w * 128;                                       // this warp's slice of every R row
-  for (int32_t c0 = w * 128; c0 < n; c0 += CHUNK) {
+  for (int32_t c0 = col_b + w * 128; c0 < col_e; c0 += CHUNK) {
     uint32_t op[4], oq[4];
     int32_t cpt[4], cqt[4];
 #pragma unroll
@@ -205,6 +230,8 @@ __global__ void __launch_bounds__(NT, 2) k_expand(const int32_t *__restrict__ D,
       __syncwarp();
     }
   }
+  __syncthreads();   // the next item rebuilds the shared row tables
+  }
 }
 
 // P:107 along-chain rule for same-chain pairs (C8: same chain id; C9: min with |off_s - off_t|)
@@ -259,10 +286,27 @@ ear_status_t expand(const ear_plan_s *plan, const int32_t *D, int64_t ldd, int32
     EAR_CUDA_TRY(cudaFuncSetAttribute(k_expand, cudaFuncAttributeMaxDynamicSharedMemorySize, EXP_SMEM));
     g_attr_set = true;
   }
-  const unsigned grid = (unsigned)ceil_div(rows, RB);
+  static int slots = 0;   // resident CTAs per device (all B200s of a box alike)
+  if (!slots) {
+    int dev = 0, sms = 0, per = 0;
+    EAR_CUDA_TRY(cudaGetDevice(&dev));
+    EAR_CUDA_TRY(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+    EAR_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_expand, NT, EXP_SMEM));
+    slots = std::max(1, sms * std::max(per, 1));
+  }
+  const int32_t groups = (int32_t)ceil_div(rows, RB);
+  ExpandWork W{};
+  W.seg_w = (int32_t)round_up(ceil_div(plan->n, 8), CHUNK);
+  W.nseg = (int32_t)ceil_div(plan->n, W.seg_w);
+  const int32_t nsplit = std::min(groups, slots);
+  W.n_full = groups - nsplit;
+  W.n_items = W.n_full + nsplit * W.nseg;
+  EAR_CUDA_TRY(cudaMallocAsync((void **)&W.counter, sizeof(int32_t), st));
+  EAR_CUDA_TRY(cudaMemsetAsync(W.counter, 0, sizeof(int32_t), st));
+  const unsigned grid = (unsigned)std::min<int64_t>(W.n_items, slots);
   const double nr = plan->n_reduced;
   int se = prof_begin(PK_EXPAND, st);
-  EAR_LAUNCH(k_expand, grid, NT, EXP_SMEM, st)(D, ldd, plan->desc, plan->n, row_begin, row_end, out, ldo);
+  EAR_LAUNCH(k_expand, grid, NT, EXP_SMEM, st)(D, ldd, plan->desc, plan->n, row_begin, row_end, out, ldo, W);
   prof_end(se, st, 4.0 * rows * plan->n + 16.0 * plan->n + 4.0 * nr * nr * rows / plan->n);
   if (plan->n_chain_vertices > 0) {
     int ss = prof_begin(PK_SAME_CHAIN, st);
@@ -271,6 +315,7 @@ ear_status_t expand(const ear_plan_s *plan, const int32_t *D, int64_t ldd, int32
                                       row_end, out, ldo);
     prof_end(ss, st, 0);
   }
+  cudaFreeAsync(W.counter, st);
   EAR_CUDA_TRY(cudaGetLastError());
   return EAR_OK;
 }

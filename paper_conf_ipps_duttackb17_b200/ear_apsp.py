@@ -61,7 +61,8 @@ class _Profile(ctypes.Structure):
 class _BccInfo(ctypes.Structure):
     _fields_ = [("n_components", ctypes.c_int32), ("n_blocks", ctypes.c_int32), ("n_articulation", ctypes.c_int32),
                 ("n_pieces", ctypes.c_int32), ("largest_piece", ctypes.c_int32), ("tree_levels", ctypes.c_int32),
-                ("sum_cubes", ctypes.c_double)]
+                ("sum_cubes", ctypes.c_double), ("rereduced_pieces", ctypes.c_int32), ("largest_reduced", ctypes.c_int32),
+                ("rereduce_levels", ctypes.c_int32)]
 
 
 # (name, restype, argtypes) for every symbol declared in include/ear_apsp.h
@@ -96,14 +97,15 @@ SIGNATURES = {
 
 
 def lib_path() -> str:
-    return _build.LIB
+    # EAR_LIB: another in-tree build of the same library (A/B timing in tools/); default libearapsp.so
+    return os.environ.get("EAR_LIB") or _build.LIB
 
 
 def lib():
     """Load libearapsp.so (built in-tree by __graft_entry__.build()).  Raises if it is missing."""
     global _lib
     if _lib is None:
-        path = _build.LIB
+        path = lib_path()
         if not os.path.exists(path):
             raise EarError(f"{path} is missing: run __graft_entry__.build() (no CPU fallback exists)")
         L = ctypes.CDLL(path)

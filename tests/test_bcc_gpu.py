@@ -123,6 +123,61 @@ def test_bcc_dominant_multi_tile_block(pkg, seed):
     assert_exact(run_full(pkg, g, pkg.FLAG_BCC), oracle.apsp(g.n, g.src, g.dst, g.w), f"dominant {seed}")
 
 
+def decorated_grid(side, frac, seed):
+    """A side x side grid block whose edges are, with probability frac, subdivided by a vertex x that
+    also carries a pendant triangle: x has degree 3 in G (a terminal of G^r) but degree 2 inside the
+    grid block, so the block reduces again (some edges get a second subdivision of plain degree-two
+    vertices, some pendants get a pendant path).  Random weights 1-100, random relabelling."""
+    rng = np.random.default_rng(seed)
+    us, vs = [], []
+    n = side * side
+    for y in range(side):
+        for x in range(side):
+            i = y * side + x
+            for j in ([i + 1] if x + 1 < side else []) + ([i + side] if y + 1 < side else []):
+                if rng.random() < frac:
+                    xv, a, b = n, n + 1, n + 2
+                    n += 3
+                    us += [i, xv, xv, a, b]
+                    vs += [xv, j, a, b, xv]
+                    if rng.random() < 0.3:   # a plain chain vertex on the other half-edge too
+                        us[-4] = n
+                        us.append(n); vs.append(xv)
+                        n += 1
+                else:
+                    us.append(i); vs.append(j)
+    perm = rng.permutation(n)
+    src = perm[np.array(us)].astype(np.int32)
+    dst = perm[np.array(vs)].astype(np.int32)
+    w = rng.integers(1, 101, len(src)).astype(np.int32)
+    return gg.Graph(n, src, dst, w)
+
+
+@pytest.mark.parametrize("seed", range(3))
+def test_bcc_rereduce_big_pieces(pkg, seed, monkeypatch):
+    """P:123's order -- G split into blocks, then EACH block reduced: a subdividing vertex with a
+    hanging triangle is a terminal of G^r but has degree two inside its block, so the big piece is
+    reduced again (possibly twice) and expanded back.  The composed D equals the FW on the whole piece
+    (EAR_NO_REREDUCE) bit for bit, and the full S equals the oracle."""
+    g = decorated_grid(24 + 4 * seed, 0.3 + 0.1 * seed, seed)
+    plan = pkg.ear_decompose(g.n, dev(g.src), dev(g.dst), dev(g.w), flags=pkg.FLAG_BCC)
+    D = pkg.alloc_D(plan)
+    pkg.apsp_reduced(plan, D)
+    torch.cuda.synchronize()
+    info = plan.bcc_info()
+    assert info["rereduced_pieces"] >= 1 and 0 < info["largest_reduced"] < info["largest_piece"] - 128, info
+    assert info["rereduce_levels"] >= 1
+    with monkeypatch.context() as m:
+        m.setenv("EAR_NO_REREDUCE", "1")
+        p2 = pkg.ear_decompose(g.n, dev(g.src), dev(g.dst), dev(g.w), flags=pkg.FLAG_BCC)
+        D2 = pkg.alloc_D(p2)
+        pkg.apsp_reduced(p2, D2)
+        torch.cuda.synchronize()
+        assert p2.bcc_info()["rereduced_pieces"] == 0
+    assert torch.equal(D, D2)
+    assert_exact(run_full(pkg, g, pkg.FLAG_BCC), oracle.apsp(g.n, g.src, g.dst, g.w), f"rereduce {seed}")
+
+
 @pytest.mark.parametrize("name", ["cfg1", "cfg2", "block"])
 def test_bcc_D_equals_fw_D(pkg, name):
     """Composed S^r (pieces + P:131 join) equals the blocked-FW S^r bit for bit, padding included."""
@@ -145,6 +200,10 @@ def test_bcc_cfg4_sampled_rows(pkg):
     print("cfg4 bcc", info, file=sys.stderr)
     D = pkg.alloc_D(plan)
     pkg.apsp_reduced(plan, D)
+    torch.cuda.synchronize()
+    info = plan.bcc_info()
+    print("cfg4 bcc after solve", info, file=sys.stderr)
+    assert info["rereduced_pieces"] >= 1 and info["largest_reduced"] < info["largest_piece"]
     rows = np.unique(np.concatenate([[0, g.n - 1], np.random.default_rng(9).choice(g.n, 24, replace=False)]))
     out = torch.empty((len(rows), g.n), dtype=torch.int32, device="cuda")
     for i, r in enumerate(rows):

@@ -23,7 +23,8 @@ torch.cuda.set_device(0)
 dist.init_process_group("nccl", rank=0, world_size=1, device_id=torch.device("cuda", 0))
 comm = ea.Comm.from_torch_distributed()
 dev = lambda a: torch.as_tensor(np.ascontiguousarray(a, dtype=np.int32)).cuda()
-for g in [gg.config("cfg1"), gg.corner_cases(12, n_target=500)]:
+from tests.test_bcc_gpu import decorated_grid   # a big piece that FLAG_BCC reduces again
+for g in [gg.config("cfg1"), gg.corner_cases(12, n_target=500), decorated_grid(24, 0.3, 0)]:
     ref = oracle.apsp(g.n, g.src, g.dst, g.w)
     for flags in (0, ea.FLAG_SSSP, ea.FLAG_BCC, ea.FLAG_FW32, ea.FLAG_BCC | ea.FLAG_FW32):
         out = ea.apsp_full(g.n, dev(g.src), dev(g.dst), dev(g.w), comm=comm, flags=flags)
