@@ -253,6 +253,10 @@ typedef struct {
   double fw16_conv_ms;         /* 16-bit path: int32 <-> u16 conversions and the range check */
   double fw_phase3_16_ms;      /* the part of fw_phase3_ms spent in the packed 16-bit tile kernel */
   double fw_phase3_16_minplus; /* its algorithmic min-plus (two per VIADDMNMX.U16x2) */
+  double fw_side_ms;           /* packed FW lookahead: phases 1-2 of round k+1 on the side stream, timed
+                                  there -- they OVERLAP phase 3 of round k, so this is not additive */
+  double rereduce_ms;          /* EAR_FLAG_BCC: Phase I + Phase III of re-reduced big pieces */
+  double bcc_prepare_ms;       /* EAR_FLAG_BCC: block structure of G^r (first solve of a plan only) */
 } ear_profile_t;
 
 void ear_profile_enable(int32_t on);

@@ -703,7 +703,9 @@ static ear_status_t reduce_solve(const ear_plan_s *p, int32_t n, int64_t m, cons
   *done = false;
   ear_plan_s *q = new ear_plan_s;
   q->device = p->device;
+  int sr = prof_begin(PK_REREDUCE, st);
   ear_status_t s = decompose(n, m, u, v, w, p->flags & EAR_FLAG_FW32, st, q);
+  prof_end(sr, st, 0);
   // worth it when the FW runs on fewer 128-tiles (same tile count: same FW work, plus the expansion)
   const int64_t unit = (int64_t)TILE * (comm ? comm->nranks : 1);
   const bool worth = s == EAR_OK && round_up(std::max<int64_t>(q->n_reduced, 1), unit) < round_up(n, unit);
@@ -746,7 +748,7 @@ static ear_status_t reduce_solve(const ear_plan_s *p, int32_t n, int64_t m, cons
       if (S) cudaFreeAsync(S, st);
     }
   }
-  if (s == EAR_OK) s = expand(q, D, Np, 0, n, M, ld, st);
+  if (s == EAR_OK) s = expand(q, D, Np, 0, n, M, ld, st, PK_REREDUCE);
   if (D) cudaFreeAsync(D, st);
   cudaStreamSynchronize(st);   // q's arrays are freed below
   plan_free(q);
@@ -789,7 +791,10 @@ static ear_status_t piece_rereduce(ear_plan_s *p, ear_bcc_s *b, int32_t id, int3
 ear_status_t bcc_solve(ear_plan_s *p, ear_comm_s *comm, int32_t *D, int64_t ldd, int32_t Np, int32_t row0,
                        int32_t rows, const int32_t *d_tile_rows, cudaStream_t st) {
   const int32_t P = comm ? comm->nranks : 1;
-  EAR_TRY(bcc_prepare(p, P, st));
+  int sb = prof_begin(PK_BCC_PREP, st);
+  ear_status_t sprep = bcc_prepare(p, P, st);
+  prof_end(sb, st, 0);
+  EAR_TRY(sprep);
   ear_bcc_s *b = p->bcc;
   const int32_t nr = p->n_reduced;
   int32_t *pool = nullptr;

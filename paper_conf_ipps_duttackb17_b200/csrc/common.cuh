@@ -88,7 +88,7 @@ struct ear_comm_s {
 namespace ear {
 // prof.cu
 enum ProfKind { PK_DECOMPOSE, PK_FW_INIT, PK_FW_P1, PK_FW_P2, PK_FW_P3, PK_COMM, PK_EXPAND, PK_SAME_CHAIN, PK_SSSP, PK_BCC, PK_COMPOSE,
-                PK_FW_P3_16, PK_FW16_CONV };
+                PK_FW_P3_16, PK_FW16_CONV, PK_FW_SIDE_P1, PK_FW_SIDE_P2, PK_REREDUCE, PK_BCC_PREP };
 void prof_fw16(bool used);   // one 16-bit FW attempt: used, or fell back to int32
 void count_launch(int n = 1);
 int prof_begin(int kind, cudaStream_t s);                // -1 when profiling is off
@@ -130,7 +130,7 @@ ear_status_t bcc_solve(ear_plan_s *plan, ear_comm_s *comm, int32_t *D, int64_t l
 void bcc_free(ear_bcc_s *b, cudaStream_t stream);
 // expand.cu
 ear_status_t expand(const ear_plan_s *plan, const int32_t *D, int64_t ldd, int32_t row_begin,
-                    int32_t row_end, int32_t *out, int64_t ldo, cudaStream_t stream);
+                    int32_t row_end, int32_t *out, int64_t ldo, cudaStream_t stream, int prof_kind = PK_EXPAND);
 ear_status_t query_pairs(const ear_plan_s *plan, const int32_t *D, int64_t ldd, int64_t npairs, const int32_t *qs,
                          const int32_t *qt, int32_t *out, cudaStream_t stream);
 // comm.cu

@@ -279,7 +279,7 @@ bool g_attr_set = false;
 }  // namespace
 
 ear_status_t expand(const ear_plan_s *plan, const int32_t *D, int64_t ldd, int32_t row_begin, int32_t row_end,
-                    int32_t *out, int64_t ldo, cudaStream_t st) {
+                    int32_t *out, int64_t ldo, cudaStream_t st, int prof_kind) {
   const int32_t rows = row_end - row_begin;
   if (rows <= 0) return EAR_OK;
   if (!g_attr_set) {
@@ -305,11 +305,11 @@ ear_status_t expand(const ear_plan_s *plan, const int32_t *D, int64_t ldd, int32
   EAR_CUDA_TRY(cudaMemsetAsync(W.counter, 0, sizeof(int32_t), st));
   const unsigned grid = (unsigned)std::min<int64_t>(W.n_items, slots);
   const double nr = plan->n_reduced;
-  int se = prof_begin(PK_EXPAND, st);
+  int se = prof_begin(prof_kind, st);
   EAR_LAUNCH(k_expand, grid, NT, EXP_SMEM, st)(D, ldd, plan->desc, plan->n, row_begin, row_end, out, ldo, W);
   prof_end(se, st, 4.0 * rows * plan->n + 16.0 * plan->n + 4.0 * nr * nr * rows / plan->n);
   if (plan->n_chain_vertices > 0) {
-    int ss = prof_begin(PK_SAME_CHAIN, st);
+    int ss = prof_begin(prof_kind == PK_EXPAND ? PK_SAME_CHAIN : prof_kind, st);
     const int g2 = (int)std::min<int64_t>(ceil_div((int64_t)rows * 32, 256), 148 * 16);
     EAR_LAUNCH(k_same_chain, g2, 256, 0, st)(plan->desc, plan->seg_of, plan->seg_start, plan->seg_vert, row_begin,
                                       row_end, out, ldo);

@@ -1017,10 +1017,11 @@ ear_status_t fw_single16(int32_t *D, int64_t ldd, int32_t Np, const int32_t *lab
   auto pivot = [&](int k, cudaStream_t q) -> ear_status_t {
     uint16_t *P16 = D16 + (int64_t)k * TILE * Np;
     uint32_t *Pk = Pd + (size_t)(k & 1) * TILE * Np;
-    int s1 = prof_begin(PK_FW_P1, q);
+    const bool on_side = q != st;   // lookahead: overlapped with phase 3, reported apart
+    int s1 = prof_begin(on_side ? PK_FW_SIDE_P1 : PK_FW_P1, q);
     EAR_LAUNCH(k_fw_phase1_16, 1, NT, 0, q)(P16 + (int64_t)k * TILE, Np);
     prof_end(s1, q, tile_ops);
-    int s2 = prof_begin(PK_FW_P2, q);
+    int s2 = prof_begin(on_side ? PK_FW_SIDE_P2 : PK_FW_P2, q);
     EAR_LAUNCH(k_dup16, grid_for(ndup), 256, 0, q)(P16, Np, Pk);   // B of phase 2: the pre-phase-2 row
     TileJob16 J{D16, Np, k * TILE, k, nt, MODE_PIVOT_ROW, 1, 0};
     EAR_TRY(launch16<Fw16Tile>(mA, mB[k & 1], J, nt - 1, q));

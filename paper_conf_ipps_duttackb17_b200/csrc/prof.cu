@@ -103,6 +103,12 @@ ear_status_t ear_profile_read(ear_profile_t *out) {
         g_acc.fw_phase3_16_ms += ms; g_acc.fw_phase3_16_minplus += r.work;
         break;
       case PK_FW16_CONV: g_acc.fw16_conv_ms += ms; break;
+      case PK_FW_SIDE_P1: g_acc.fw_side_ms += ms; g_acc.fw_phase1_launches++; break;
+      case PK_FW_SIDE_P2:
+        g_acc.fw_side_ms += ms; g_acc.fw_phase2_launches++; g_acc.fw_phase2_minplus += r.work;
+        break;
+      case PK_REREDUCE: g_acc.rereduce_ms += ms; break;
+      case PK_BCC_PREP: g_acc.bcc_prepare_ms += ms; break;
       default: break;
     }
     g_pool.push_back(r.e0);

@@ -55,7 +55,8 @@ class _Profile(ctypes.Structure):
                 ("sssp_arcs", ctypes.c_double), ("bcc_pieces_ms", ctypes.c_double), ("compose_ms", ctypes.c_double),
                 ("compose_bytes", ctypes.c_double), ("fw16_used", ctypes.c_int64), ("fw16_fallbacks", ctypes.c_int64),
                 ("fw16_conv_ms", ctypes.c_double), ("fw_phase3_16_ms", ctypes.c_double),
-                ("fw_phase3_16_minplus", ctypes.c_double)]
+                ("fw_phase3_16_minplus", ctypes.c_double), ("fw_side_ms", ctypes.c_double),
+                ("rereduce_ms", ctypes.c_double), ("bcc_prepare_ms", ctypes.c_double)]
 
 
 class _BccInfo(ctypes.Structure):
