@@ -143,6 +143,16 @@ ear_status_t apsp_reduced(ear_plan_t plan, int32_t *d_D, int64_t ldd, ear_comm_t
 ear_status_t apsp_reduced_emulated(ear_plan_t plan, int32_t nranks, int32_t *d_D, int64_t ldd,
                                    void *stream);
 
+/* DIAGNOSTIC, produces no result: the device work of ONE rank `rank` of an `nranks`-rank run of the
+ * packed 16-bit sharded FW (sec. 7 of DESIGN.md) on the current device -- narrowing its owned rows,
+ * and per round the pivot-row widening, the int32 phases 1-2, the narrowing and the packed phase 3 on
+ * its owned upper tiles -- without the other ranks and without the exchange (the pivot row block then
+ * holds only this rank's pieces; min-plus work is data-independent, so the time is that rank's
+ * compute).  Used to measure per-rank compute scaling on one GPU (tools/rank_timing.py).  Allocates
+ * and frees its own scratch; asynchronous.  Errors: EAR_EINVAL (NULL plan, rank out of range),
+ * EAR_ENOMEM, EAR_ECUDA. */
+ear_status_t apsp_reduced_rank_timing(ear_plan_t plan, int32_t nranks, int32_t rank, void *stream);
+
 /* Number of 128-row tile blocks a rank owns under the sharded layout of apsp_reduced (Np =
  * ear_plan_info(nranks).n_reduced_padded).  Host-only. */
 int32_t ear_owned_tile_rows(int32_t n_reduced_padded, int32_t nranks, int32_t rank);

@@ -212,6 +212,15 @@ ear_status_t apsp_reduced_emulated(ear_plan_t p, int32_t nranks, int32_t *d_D, i
   return fw_sharded_emulated(p, d_D, ldd, Np, nranks, (cudaStream_t)stream);
 }
 
+ear_status_t apsp_reduced_rank_timing(ear_plan_t p, int32_t nranks, int32_t rank, void *stream) {
+  g_err[0] = 0;
+  if (!p || nranks < 1 || rank < 0 || rank >= nranks) {
+    set_error("apsp_reduced_rank_timing: bad argument");
+    return EAR_EINVAL;
+  }
+  return fw_rank_timing(p, padded(p, nranks), nranks, rank, (cudaStream_t)stream);
+}
+
 int32_t ear_owned_tile_rows(int32_t n_reduced_padded, int32_t nranks, int32_t rank) {
   if (nranks < 1 || rank < 0 || rank >= nranks) return 0;
   return shard_nown(n_reduced_padded / TILE, nranks, rank);

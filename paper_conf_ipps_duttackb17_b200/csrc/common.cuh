@@ -113,6 +113,7 @@ ear_status_t fw_sharded_auto(int32_t *S, int64_t ldd, int32_t Np, ear_comm_s *co
                              int32_t n_real, bool allow16, cudaStream_t stream);
 ear_status_t fw_sharded_gather(const int32_t *S, int64_t ldd, int32_t Np, int32_t *Df, int64_t ldf, ear_comm_s *comm,
                                cudaStream_t stream);
+ear_status_t fw_rank_timing(const ear_plan_s *plan, int32_t Np, int32_t P, int32_t rank, cudaStream_t stream);
 ear_status_t fw_sharded_emulated(ear_plan_s *plan, int32_t *D, int64_t ldd, int32_t Np, int32_t P,
                                  cudaStream_t stream);
 int32_t shard_nown(int32_t nt, int32_t P, int32_t rank);

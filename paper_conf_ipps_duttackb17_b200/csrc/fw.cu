@@ -19,6 +19,7 @@
 #include <cudaTypedefs.h>
 
 #include <algorithm>
+#include <cstdio>
 #include <cstdlib>
 #include <cmath>
 #include <vector>
@@ -173,6 +174,20 @@ __device__ __forceinline__ bool mbar_try(uint64_t *b, uint32_t parity) {
 }
 __device__ __forceinline__ void mbar_wait(uint64_t *b, uint32_t parity) {
   while (!mbar_try(b, parity)) {
+  }
+}
+// non-suspending poll (test_wait): the warp stays resident and issuing while it waits
+__device__ __forceinline__ bool mbar_test(uint64_t *b, uint32_t parity) {
+  uint32_t ok;
+  asm volatile(
+      "{\n\t.reg .pred p;\n\tmbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\n\tselp.u32 %0, 1, 0, p;\n\t}\n"
+      : "=r"(ok)
+      : "r"(smem_u32(b)), "r"(parity)
+      : "memory");
+  return ok != 0;
+}
+__device__ __forceinline__ void mbar_wait_spin(uint64_t *b, uint32_t parity) {
+  while (!mbar_test(b, parity)) {
   }
 }
 __device__ __forceinline__ void tma_load_2d(void *dst, const CUtensorMap *map, int32_t c0, int32_t c1, uint64_t *bar) {
@@ -337,36 +352,42 @@ __global__ void k_fill(int32_t *p, int64_t n, int32_t v) {
 // Pivot-row block <-> a rank's owned storage, round k (prow: 128 x Np, leading dimension Np).
 //   dir = 0 (gather):  prow[:, ti-block] = S(ti, k)^T for owned ti < k; prow[:, j >= k] = S(k, j) if row k owned
 //   dir = 1 (scatter): the inverse, after phases 1 and 2 updated prow
-// grid: (16 sub-blocks of 32 x 32, Np/128 column tiles, nown owned rows), 256 threads
-__global__ void k_prow_xfer(int32_t *S, int64_t ldd, const int32_t *orow, int32_t k, int32_t *prow, int32_t Np,
-                            int dir) {
-  __shared__ int32_t t[32][33];
-  const int lr = blockIdx.z, ti = orow[lr], tj = blockIdx.y;
+// Only the pieces are launched: grid (16 sub-blocks of 32 x 32, npieces), 256 threads, where pieces
+// [0, nrow) are the tiles j = k + y of the pivot row when this rank owns it (nrow = nt - k, local row
+// posk) and the next mk are the owned rows ti < k (the first mk owned rows: ascending), tile (ti, k).
+// TS / TP: storage / block element types (int32 <-> int32; u16 -> int32 to assemble the packed
+// schedule's exchange block, u16 -> u16 to scatter its narrowed block back).
+template <class TS, class TP>
+__global__ void k_prow_xfer(TS *S, int64_t ldd, const int32_t *orow, int32_t k, int32_t nt, int32_t posk, TP *prow,
+                            int32_t Np, int dir) {
+  __shared__ uint32_t t[32][33];
+  const int nrow = posk >= 0 ? nt - k : 0;
+  const int y = blockIdx.y;
   const int bx = blockIdx.x & 3, by = blockIdx.x >> 2;         // 32 x 32 sub-block (bx: x, by: y)
   const int lx = threadIdx.x & 31, ly = threadIdx.x >> 5;      // 32 x 8 threads
-  if (ti == k) {               // the pivot row's upper part: plain copy, tiles j >= k
-    if (tj < k) return;
+  if (y < nrow) {              // the pivot row's upper part: plain copy, tiles j >= k
+    const int lr = posk, tj = k + y;
     for (int yy = ly; yy < 32; yy += 8) {
       const int64_t row = by * 32 + yy, col = (int64_t)tj * TILE + bx * 32 + lx;
-      int32_t *s = S + ((int64_t)lr * TILE + row) * ldd + col;
-      int32_t *p = prow + row * Np + col;
-      if (dir == 0) *p = *s; else *s = *p;
+      TS *sp = S + ((int64_t)lr * TILE + row) * ldd + col;
+      TP *pp = prow + row * Np + col;
+      if (dir == 0) *pp = (TP)*sp; else *sp = (TS)*pp;
     }
     return;
   }
-  if (ti > k || tj != k) return;   // owned row below the pivot: its tile (ti, k) <-> prow[:, ti-block]^T
+  const int lr = y - nrow, ti = orow[lr];   // owned row below the pivot: tile (ti, k) <-> prow[:, ti-block]^T
   if (dir == 0) {
     for (int yy = ly; yy < 32; yy += 8)   // S rows ti-block (bx*32+yy), cols k-block (by*32+lx)
-      t[yy][lx] = S[((int64_t)lr * TILE + bx * 32 + yy) * ldd + (int64_t)k * TILE + by * 32 + lx];
+      t[yy][lx] = (uint32_t)S[((int64_t)lr * TILE + bx * 32 + yy) * ldd + (int64_t)k * TILE + by * 32 + lx];
     __syncthreads();
     for (int yy = ly; yy < 32; yy += 8)   // prow rows (by*32+yy), cols ti-block (bx*32+lx)
-      prow[(int64_t)(by * 32 + yy) * Np + (int64_t)ti * TILE + bx * 32 + lx] = t[lx][yy];
+      prow[(int64_t)(by * 32 + yy) * Np + (int64_t)ti * TILE + bx * 32 + lx] = (TP)t[lx][yy];
   } else {
     for (int yy = ly; yy < 32; yy += 8)
-      t[yy][lx] = prow[(int64_t)(by * 32 + yy) * Np + (int64_t)ti * TILE + bx * 32 + lx];
+      t[yy][lx] = (uint32_t)prow[(int64_t)(by * 32 + yy) * Np + (int64_t)ti * TILE + bx * 32 + lx];
     __syncthreads();
     for (int yy = ly; yy < 32; yy += 8)
-      S[((int64_t)lr * TILE + bx * 32 + yy) * ldd + (int64_t)k * TILE + by * 32 + lx] = t[lx][yy];
+      S[((int64_t)lr * TILE + bx * 32 + yy) * ldd + (int64_t)k * TILE + by * 32 + lx] = (TS)t[lx][yy];
   }
 }
 
@@ -480,43 +501,8 @@ __global__ void k_from16r(const uint16_t *__restrict__ S16, int64_t ld16, int32_
   }
 }
 
-// k_prow_xfer for a 16-bit owned storage: dir 0 gathers S16 pieces into the int32 exchange block
-// (u16 -> int32; C16 < INF, so the MIN all-reduce keeps it), dir 1 scatters the capped 16-bit pivot
-// row block back.  Same grid and piece rule as k_prow_xfer.
-template <class TP>
-__global__ void k_prow_xfer16(uint16_t *S, int64_t ldd, const int32_t *orow, int32_t k, TP *prow, int32_t Np, int dir) {
-  __shared__ uint32_t t[32][33];
-  const int lr = blockIdx.z, ti = orow[lr], tj = blockIdx.y;
-  const int bx = blockIdx.x & 3, by = blockIdx.x >> 2;
-  const int lx = threadIdx.x & 31, ly = threadIdx.x >> 5;
-  if (ti == k) {
-    if (tj < k) return;
-    for (int yy = ly; yy < 32; yy += 8) {
-      const int64_t row = by * 32 + yy, col = (int64_t)tj * TILE + bx * 32 + lx;
-      uint16_t *s = S + ((int64_t)lr * TILE + row) * ldd + col;
-      TP *p = prow + row * Np + col;
-      if (dir == 0) *p = (TP)*s; else *s = (uint16_t)*p;
-    }
-    return;
-  }
-  if (ti > k || tj != k) return;
-  if (dir == 0) {
-    for (int yy = ly; yy < 32; yy += 8)
-      t[yy][lx] = S[((int64_t)lr * TILE + bx * 32 + yy) * ldd + (int64_t)k * TILE + by * 32 + lx];
-    __syncthreads();
-    for (int yy = ly; yy < 32; yy += 8)
-      prow[(int64_t)(by * 32 + yy) * Np + (int64_t)ti * TILE + bx * 32 + lx] = (TP)t[lx][yy];
-  } else {
-    for (int yy = ly; yy < 32; yy += 8)
-      t[yy][lx] = (uint32_t)prow[(int64_t)(by * 32 + yy) * Np + (int64_t)ti * TILE + bx * 32 + lx];
-    __syncthreads();
-    for (int yy = ly; yy < 32; yy += 8)
-      S[((int64_t)lr * TILE + bx * 32 + yy) * ldd + (int64_t)k * TILE + by * 32 + lx] = (uint16_t)t[lx][yy];
-  }
-}
-
-// the pivot row block after the int32 phases 1-2 -> its capped u16 copy (A operand, scattered back to
-// the owners) and the duplicated u32 copy (B operand); n = TILE * Np, n % 4 == 0
+// the assembled int32 pivot row block -> its capped u16 copy and (Pd non-null) the duplicated u32 copy;
+// n = TILE * Np, n % 4 == 0
 __global__ void k_prow_to16(const int32_t *__restrict__ P32, uint16_t *__restrict__ P16, uint32_t *__restrict__ Pd,
                             int64_t n) {
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n / 4; i += (int64_t)gridDim.x * blockDim.x) {
@@ -524,7 +510,7 @@ __global__ void k_prow_to16(const int32_t *__restrict__ P32, uint16_t *__restric
     const uint32_t a = (uint32_t)min(v.x, (int32_t)C16), b = (uint32_t)min(v.y, (int32_t)C16);
     const uint32_t c = (uint32_t)min(v.z, (int32_t)C16), d = (uint32_t)min(v.w, (int32_t)C16);
     reinterpret_cast<uint2 *>(P16)[i] = make_uint2(a | (b << 16), c | (d << 16));
-    reinterpret_cast<uint4 *>(Pd)[i] = make_uint4(a * 0x10001u, b * 0x10001u, c * 0x10001u, d * 0x10001u);
+    if (Pd) reinterpret_cast<uint4 *>(Pd)[i] = make_uint4(a * 0x10001u, b * 0x10001u, c * 0x10001u, d * 0x10001u);
   }
 }
 
@@ -624,24 +610,27 @@ struct TileJob16 {
   const int32_t *orow;
   const int64_t *opre;
   int32_t nown, mk, posk;
+  unsigned long long *dbg;   // development (EAR_FW16_DBG): per-CTA %globaltimer at start / end, or null
+  int32_t ti0;               // first tile row held by C (MODE_PIVOT_ROW on a standalone pivot row block: k)
 };
 
 // LAR = 1: a ring stage is refilled by the LAST warp to finish consuming it (a shared counter) instead
 // of thread 0 waiting on an 'empty' barrier at the start of each chunk (which ties warp 0 to the
 // slowest warp every chunk).
-template <int KC, int STAGES, int MINB, int UNR, int NTH = 256, int PFC = 0, int LAR = 0>
+template <int KC, int STAGES, int MINB, int UNR, int NTH = 256, int PFC = 0, int LAR = 0, int SPIN = 0>
 struct Fw16Cfg {
   static constexpr int NCHUNK = TILE / KC;
   static constexpr int A_CHUNK = KC * TILE;   // u16 elements
   static constexpr int B_CHUNK = KC * TILE;   // u32 elements
   static constexpr int SMEM = STAGES * (A_CHUNK * 2 + B_CHUNK * 4) + 2 * STAGES * 8 + STAGES * 4;
   static constexpr int kKC = KC, kSTAGES = STAGES, kMINB = MINB, kUNR = UNR, kNTH = NTH, kPFC = PFC, kLAR = LAR;
+  static constexpr int kSPIN = SPIN;
   static constexpr int RPH = 256 * 2 / NTH;   // row pairs per 64-row half owned by a thread (2 or 4)
 };
 
 __device__ __forceinline__ void decode16(const TileJob16 &J, int64_t idx, int &ti, int &tj, int &lr) {
   TileJob T{};
-  T.k = J.k; T.nt = J.nt; T.mode = J.mode; T.ti0 = 0;
+  T.k = J.k; T.nt = J.nt; T.mode = J.mode; T.ti0 = J.ti0;
   T.orow = J.orow; T.opre = J.opre; T.nown = J.nown; T.mk = J.mk; T.posk = J.posk;
   decode_tile(T, idx, ti, tj, lr);
 }
@@ -661,6 +650,14 @@ __global__ void __launch_bounds__(CF::kNTH, CF::kMINB)
   int32_t *cnt = reinterpret_cast<int32_t *>(empty + STAGES);   // LAR: warps done with the stage
   const int tid = threadIdx.x, lane = tid & 31;
   const int tx = tid & 15, ty = tid >> 4;
+  if (J.dbg && tid == 0) {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    uint32_t smid;
+    asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+    J.dbg[3 * blockIdx.x] = t;
+    J.dbg[3 * blockIdx.x + 2] = smid;
+  }
 
   const int my_tiles = J.ntiles > (int64_t)blockIdx.x ? (int)((J.ntiles - 1 - blockIdx.x) / gridDim.x + 1) : 0;
   const int total_chunks = my_tiles * NCHUNK;
@@ -738,7 +735,8 @@ __global__ void __launch_bounds__(CF::kNTH, CF::kMINB)
     for (int kc = 0; kc < NCHUNK; ++kc, ++g) {
       if (!CF::kLAR && tid == 0) produce(g + STAGES < total_chunks ? g + STAGES : total_chunks);
       const int st = g % STAGES;
-      mbar_wait(&full[st], (uint32_t)((g / STAGES) & 1));
+      if (CF::kSPIN) mbar_wait_spin(&full[st], (uint32_t)((g / STAGES) & 1));
+      else mbar_wait(&full[st], (uint32_t)((g / STAGES) & 1));
       const uint16_t *a_s = sA + st * CF::A_CHUNK;
       const uint32_t *b_s = sB + st * CF::B_CHUNK;
 #pragma unroll CF::kUNR
@@ -804,6 +802,14 @@ __global__ void __launch_bounds__(CF::kNTH, CF::kMINB)
           }
         }
       }
+    }
+  }
+  if (J.dbg) {
+    __syncthreads();
+    if (tid == 0) {
+      unsigned long long t;
+      asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+      J.dbg[3 * blockIdx.x + 1] = t;
     }
   }
 }
@@ -909,6 +915,8 @@ using Fw16TileL4 = Fw16Cfg<16, 4, 3, 16, 128, 0, 1>;
 using Fw16TileL3 = Fw16Cfg<32, 3, 3, 16, 128, 0, 1>;
 using Fw16TileLP = Fw16Cfg<32, 2, 3, 16, 128, 1, 1>;
 using Fw16TileL3P = Fw16Cfg<32, 3, 3, 16, 128, 1, 1>;
+using Fw16TileS = Fw16Cfg<32, 2, 3, 16, 128, 1, 1, 1>;
+using Fw16TileS3 = Fw16Cfg<32, 3, 3, 16, 128, 1, 1, 1>;
 
 // development knobs (tools/): EAR_FW16_LOOKAHEAD=0 disables the lookahead, EAR_FW16_RESERVE sets the
 // CTA slots the rest-of-round launch leaves free for the next round's pivot work (default 0: measured
@@ -931,7 +939,23 @@ ear_status_t launch16_cfg(const CUtensorMap &mA, const CUtensorMap &mB, TileJob1
   if (per_sm < 1) per_sm = 1;
   J.ntiles = nblocks;
   const int64_t grid = std::min<int64_t>(nblocks, std::max<int64_t>(1, (int64_t)g_num_sms * per_sm - reserve));
+  // EAR_FW16_DBG=N (development): per-CTA start / end times and SM of the N-th launch, to stderr
+  static const int dbg_at = env_int("EAR_FW16_DBG", -1);
+  static int nlaunch = 0;
+  const bool dbg = dbg_at >= 0 && nlaunch++ == dbg_at;
+  if (dbg) EAR_CUDA_TRY(cudaMalloc((void **)&J.dbg, sizeof(unsigned long long) * 3 * grid));
   EAR_LAUNCH(k_fw_tiles16<CF>, (unsigned)grid, CF::kNTH, CF::SMEM, st)(mA, mB, J);
+  if (dbg) {
+    std::vector<unsigned long long> h(3 * grid);
+    EAR_CUDA_TRY(cudaStreamSynchronize(st));
+    EAR_CUDA_TRY(cudaMemcpy(h.data(), J.dbg, sizeof(unsigned long long) * 3 * grid, cudaMemcpyDeviceToHost));
+    cudaFree(J.dbg);
+    unsigned long long t0 = ~0ull;
+    for (int64_t b = 0; b < grid; ++b) t0 = std::min(t0, h[3 * b]);
+    fprintf(stderr, "FW16DBG launch %d grid %lld tiles %lld per_sm %d\n", dbg_at, (long long)grid, (long long)nblocks, per_sm);
+    for (int64_t b = 0; b < grid; ++b)
+      fprintf(stderr, "FW16DBG %lld %llu %llu %llu\n", (long long)b, h[3 * b] - t0, h[3 * b + 1] - t0, h[3 * b + 2]);
+  }
   return EAR_OK;
 }
 
@@ -949,6 +973,8 @@ ear_status_t launch16(const CUtensorMap &mA, const CUtensorMap &mB, TileJob16 J,
   if (variant == 3) return launch16_cfg<Fw16TileL3>(mA, mB, J, nblocks, st, reserve);
   if (variant == 4) return launch16_cfg<Fw16TileLP>(mA, mB, J, nblocks, st, reserve);
   if (variant == 5) return launch16_cfg<Fw16TileL3P>(mA, mB, J, nblocks, st, reserve);
+  if (variant == 6) return launch16_cfg<Fw16TileS>(mA, mB, J, nblocks, st, reserve);
+  if (variant == 7) return launch16_cfg<Fw16TileS3>(mA, mB, J, nblocks, st, reserve);
   return launch16_cfg<CF>(mA, mB, J, nblocks, st, reserve);
 }
 
@@ -1200,11 +1226,28 @@ static ear_status_t fill(int32_t *p, int64_t n, int32_t v, cudaStream_t st) {
   return EAR_OK;
 }
 
-static ear_status_t shard_xfer(const Shard &sh, int k, int32_t *prow, int dir, cudaStream_t st) {
-  if (sh.nown == 0) return EAR_OK;
-  dim3 g(16, sh.nt, sh.nown);
-  EAR_LAUNCH(k_prow_xfer, g, 256, 0, st)(sh.S, sh.ldd, sh.d_rows, k, prow, sh.Np, dir);
+// this rank's pieces of round k's pivot row block (see k_prow_xfer)
+static void shard_pieces(const Shard &sh, int k, int *posk, int *mk) {
+  *posk = -1;
+  *mk = 0;
+  for (int32_t r = 0; r < sh.nown; ++r) {
+    if (sh.rows[r] < k) ++*mk;
+    if (sh.rows[r] == k) *posk = r;
+  }
+}
+
+template <class TS, class TP>
+static ear_status_t shard_xfer_t(const Shard &sh, TS *S, int64_t ld, int k, TP *prow, int dir, cudaStream_t st) {
+  int posk, mk;
+  shard_pieces(sh, k, &posk, &mk);
+  const int np = (posk >= 0 ? sh.nt - k : 0) + mk;
+  if (np == 0) return EAR_OK;
+  EAR_LAUNCH((k_prow_xfer<TS, TP>), dim3(16, np), 256, 0, st)(S, ld, sh.d_rows, k, sh.nt, posk, prow, sh.Np, dir);
   return EAR_OK;
+}
+
+static ear_status_t shard_xfer(const Shard &sh, int k, int32_t *prow, int dir, cudaStream_t st) {
+  return shard_xfer_t<int32_t, int32_t>(sh, sh.S, sh.ldd, k, prow, dir, st);
 }
 
 // phases 1 and 2 on the assembled pivot row block
@@ -1268,10 +1311,11 @@ ear_status_t fw_sharded(int32_t *S, int64_t ldd, int32_t Np, ear_comm_s *comm, c
 // ---------------------------------------------------------------- 16-bit row-block sharding
 // The sharded schedule above on packed 16-bit owned rows (the cap C16 and its exactness argument are
 // those of fw_single16).  The exchange stays int32 -- NCCL has no 16-bit MIN: the owned u16 pieces are
-// widened into the INF-filled int32 pivot row block, all-reduced, closed by the int32 phases 1-2 (on
-// capped inputs; min(x, C16) of their result is still exact, as the cap commutes with every
-// relaxation), then narrowed into the u16 A operand (also scattered back to the owners) and the
-// duplicated u32 B operand of the packed phase-3 kernel, which updates the owned u16 rows (MODE_LIST).
+// widened into the INF-filled int32 pivot row block and all-reduced; the block is narrowed back to u16
+// (values <= C16, so exactly the capped values) and closed by the packed phases 1-2 of fw_single16's
+// pivot() -- phase 1 on the pivot tile, phase 2 as one product against the duplicated pre-phase-2 row --
+// then scattered back to the owners; its duplicated copy is the B operand of the packed phase-3
+// kernel, which updates the owned u16 rows (MODE_LIST).
 // comm == nullptr: the shards are virtual ranks on this device sharing the block (their pieces are
 // disjoint, so no exchange is needed).  The range check runs over every rank's owned upper tiles and
 // is MIN-reduced; *done = false leaves the int32 owned storage untouched for the int32 schedule.
@@ -1293,7 +1337,7 @@ static ear_status_t phase3_16(const Shard &sh, uint16_t *S16, const CUtensorMap 
 }
 
 static ear_status_t fw_sharded16(std::vector<Shard *> &sh, int32_t Np, ear_comm_s *comm, const int32_t *lab,
-                                 int32_t n_real, bool *done, cudaStream_t st) {
+                                 int32_t n_real, bool *done, cudaStream_t st, bool timing_only = false) {
   *done = false;
   const int nt = Np / TILE;
   if (nt < 2) return EAR_OK;
@@ -1329,9 +1373,8 @@ static ear_status_t fw_sharded16(std::vector<Shard *> &sh, int32_t Np, ear_comm_
   }
   const int KC = fw16_kc();
   const int64_t nblk = (int64_t)TILE * Np;
-  CUtensorMap map_prow, mA, mB;
-  ear_status_t s = make_map(&map_prow, prow, TILE, Np, Np, fw_kc());
-  if (s == EAR_OK) s = make_map_t(&mA, CU_TENSOR_MAP_DATA_TYPE_UINT16, 2, p16, TILE, Np, Np, KC);
+  CUtensorMap mA, mB;
+  ear_status_t s = make_map_t(&mA, CU_TENSOR_MAP_DATA_TYPE_UINT16, 2, p16, TILE, Np, Np, KC);
   if (s == EAR_OK) s = make_map_t(&mB, CU_TENSOR_MAP_DATA_TYPE_UINT32, 4, Pd, TILE, Np, Np, KC);
   if (s == EAR_OK) {
     int sc = prof_begin(PK_FW16_CONV, st);
@@ -1345,23 +1388,38 @@ static ear_status_t fw_sharded16(std::vector<Shard *> &sh, int32_t Np, ear_comm_
     s = fill(prow, nblk, INF, st);
     for (size_t r = 0; r < R && s == EAR_OK; ++r)
       if (sh[r]->nown > 0)
-        EAR_LAUNCH(k_prow_xfer16<int32_t>, dim3(16, nt, sh[r]->nown), 256, 0, st)(S16[r], Np, sh[r]->d_rows, k, prow,
-                                                                                  Np, 0);
+        s = shard_xfer_t<uint16_t, int32_t>(*sh[r], S16[r], Np, k, prow, 0, st);
     if (s == EAR_OK && comm) {
       int sc = prof_begin(PK_COMM, st);
       s = comm_allreduce_min(comm, prow, nblk, st);
       prof_end(sc, st, 0);
     }
-    if (s == EAR_OK) s = shard_pivot(prow, map_prow, Np, k, st);
     if (s != EAR_OK) break;
-    EAR_LAUNCH(k_prow_to16, grid_for(nblk / 4), 256, 0, st)(prow, p16, Pd, nblk);
+    // phases 1-2 packed, as fw_single16's pivot(): narrow, close the pivot tile, B = the pre-phase-2
+    // row duplicated, the pivot-row tiles as one product, then B again for phase 3
+    EAR_LAUNCH(k_prow_to16, grid_for(nblk / 4), 256, 0, st)(prow, p16, nullptr, nblk);
+    int s1 = prof_begin(PK_FW_P1, st);
+    EAR_LAUNCH(k_fw_phase1_16, 1, NT, 0, st)(p16 + (int64_t)k * TILE, Np);
+    prof_end(s1, st, (double)TILE * TILE * TILE);
+    int s2 = prof_begin(PK_FW_P2, st);
+    EAR_LAUNCH(k_dup16, grid_for(nblk / 4), 256, 0, st)(p16, Np, Pd);
+    TileJob16 J2{p16, Np, 0, k, nt, MODE_PIVOT_ROW, 0, 0};
+    J2.ti0 = k;
+    s = launch16<Fw16Tile>(mA, mB, J2, nt - 1, st);
+    EAR_LAUNCH(k_dup16, grid_for(nblk / 4), 256, 0, st)(p16, Np, Pd);
+    prof_end(s2, st, (double)(nt - 1) * TILE * TILE * TILE);
+    if (s != EAR_OK) break;
     for (size_t r = 0; r < R; ++r)
       if (sh[r]->nown > 0)
-        EAR_LAUNCH(k_prow_xfer16<uint16_t>, dim3(16, nt, sh[r]->nown), 256, 0, st)(S16[r], Np, sh[r]->d_rows, k, p16,
-                                                                                   Np, 1);
+        s = shard_xfer_t<uint16_t, uint16_t>(*sh[r], S16[r], Np, k, p16, 1, st);
     for (size_t r = 0; r < R && s == EAR_OK; ++r) s = phase3_16(*sh[r], S16[r], mA, mB, k, st);
   }
   int32_t h_flag = -1;
+  if (s == EAR_OK && timing_only) {   // apsp_reduced_rank_timing: no check, no result
+    release();
+    EAR_CUDA_TRY(cudaGetLastError());
+    return EAR_OK;
+  }
   if (s == EAR_OK) {
     int sc = prof_begin(PK_FW16_CONV, st);
     cudaMemsetAsync(flag, 0, sizeof(int32_t), st);
@@ -1406,6 +1464,24 @@ ear_status_t fw_sharded_auto(int32_t *S, int64_t ldd, int32_t Np, ear_comm_s *co
     if (done) return EAR_OK;
   }
   return fw_sharded(S, ldd, Np, comm, st);
+}
+
+// One rank's device work of a P-rank packed sharded FW, without the other ranks and the exchange
+// (apsp_reduced_rank_timing: per-rank compute scaling measured on one GPU).
+ear_status_t fw_rank_timing(const ear_plan_s *plan, int32_t Np, int32_t P, int32_t rank, cudaStream_t st) {
+  const size_t nown = shard_rows(Np / TILE, P, rank).size();
+  int32_t *S = nullptr;
+  EAR_CUDA_TRY(cudaMallocAsync((void **)&S, sizeof(int32_t) * std::max<size_t>(nown, 1) * TILE * Np, st));
+  Shard sh;
+  ear_status_t s = shard_setup(&sh, S, Np, Np, P, rank, st);
+  for (int32_t lr = 0; lr < sh.nown && s == EAR_OK; ++lr)
+    s = fw_init_D(plan, S + (int64_t)lr * TILE * Np, Np, Np, sh.rows[lr] * TILE, TILE, st);
+  bool done = false;
+  std::vector<Shard *> v{&sh};
+  if (s == EAR_OK) s = fw_sharded16(v, Np, nullptr, nullptr, plan->n_reduced, &done, st, true);
+  shard_free(&sh, st);
+  cudaFreeAsync(S, st);
+  return s;
 }
 
 // Full D from every rank's owned upper tiles (INF fill + scatter + all-reduce MIN).

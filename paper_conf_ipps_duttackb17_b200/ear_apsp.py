@@ -77,6 +77,7 @@ SIGNATURES = {
     "ear_bcc_info": (_I32, [_P, ctypes.POINTER(_BccInfo)]),
     "apsp_reduced": (_I32, [_P, _P, _I64, _P, _P]),
     "apsp_reduced_emulated": (_I32, [_P, _I32, _P, _I64, _P]),
+    "apsp_reduced_rank_timing": (_I32, [_P, _I32, _I32, _P]),
     "ear_owned_tile_rows": (_I32, [_I32, _I32, _I32]),
     "ear_gather_reduced": (_I32, [_P, _P, _I64, _P, _I64, _P, _P]),
     "expand_ears": (_I32, [_P, _P, _I64, _I32, _I32, _P, _I64, _P]),
@@ -266,6 +267,11 @@ def apsp_reduced_emulated(plan: Plan, nranks: int, D: torch.Tensor | None = None
     _check(lib().apsp_reduced_emulated(plan.handle, nranks, D.data_ptr(), D.stride(0), _stream(stream)),
            "apsp_reduced_emulated")
     return D
+
+
+def apsp_reduced_rank_timing(plan: Plan, nranks: int, rank: int, stream=None) -> None:
+    """Diagnostic: the device work of one rank of an nranks-rank packed sharded FW (no exchange, no result)."""
+    _check(lib().apsp_reduced_rank_timing(plan.handle, nranks, rank, _stream(stream)), "apsp_reduced_rank_timing")
 
 
 def gather_reduced(plan: Plan, D_block: torch.Tensor, comm: Comm, D_full: torch.Tensor | None = None,
