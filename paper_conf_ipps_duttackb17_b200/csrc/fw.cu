@@ -117,7 +117,9 @@ __global__ void __launch_bounds__(NT, 1) k_fw_phase1(int32_t *T, int64_t ldt) {
 // Thread 0 doubles as the TMA producer.  The C tile lives in registers (8x8 per thread).
 // MODE_CROSS / MODE_REST (single-GPU lookahead, round k): the upper tiles of row/column k+1 (without
 // column k), and all upper tiles outside rows/columns k and k+1; together they are MODE_UPPER.
-enum { MODE_PIVOT_ROW = 0, MODE_UPPER = 1, MODE_LIST = 2, MODE_CROSS = 3, MODE_REST = 4 };
+// MODE_LIST_CROSS / MODE_LIST_REST: the same split of a rank's MODE_LIST tiles (sharded lookahead).
+enum { MODE_PIVOT_ROW = 0, MODE_UPPER = 1, MODE_LIST = 2, MODE_CROSS = 3, MODE_REST = 4, MODE_LIST_CROSS = 5,
+       MODE_LIST_REST = 6 };
 
 // Tile-kernel configuration: k-chunk depth, TMA ring depth, CTAs per SM, kk-loop unroll.
 template <int KC_, int ST_, int MINB_, int UNR_>
@@ -148,6 +150,7 @@ struct TileJob {
   const int32_t *orow;
   const int64_t *opre;
   int32_t nown, mk, posk;
+  int32_t posk1;     // MODE_LIST_CROSS / _REST: position of row k+1 in the owned list or -1
 };
 
 __device__ __forceinline__ uint32_t smem_u32(const void *p) { return (uint32_t)__cvta_generic_to_shared(p); }
@@ -230,10 +233,24 @@ __device__ __forceinline__ void decode_tile(const TileJob &J, int64_t idx, int &
     lr = ti - J.ti0;
     return;
   }
+  if (J.mode == MODE_LIST_CROSS) {   // row k+1's tiles (if owned), then tile (ti, k+1) of owned rows ti < k
+    const int k1 = k + 1;
+    const int nrow = J.posk1 >= 0 ? J.nt - k1 : 0;
+    if ((int)idx < nrow) {
+      lr = J.posk1; ti = k1; tj = k1 + (int)idx;
+    } else {
+      lr = (int)idx - nrow; ti = J.orow[lr]; tj = k1;
+    }
+    return;
+  }
   // MODE_LIST: the upper tiles (ti, tj >= ti) of the owned rows, without row k and column k.
   // Per round, owned rows ti < k lose tile (ti, k) and row k (if owned) loses all its tiles.
+  // MODE_LIST_REST also drops row and column k+1 (owned rows ti < k lose two tiles).
+  const bool rest = J.mode == MODE_LIST_REST;
   auto pre = [&](int r) -> int64_t {
-    return J.opre[r] - min(r, J.mk) - ((J.posk >= 0 && r > J.posk) ? (int64_t)(J.nt - k) : 0);
+    int64_t v = J.opre[r] - (rest ? 2 : 1) * min(r, J.mk) - ((J.posk >= 0 && r > J.posk) ? (int64_t)(J.nt - k) : 0);
+    if (rest && J.posk1 >= 0 && r > J.posk1) v -= J.nt - k - 1;
+    return v;
   };
   int lo = 0, hi = J.nown - 1;   // largest r with pre(r) <= idx (ties: the last, skipping empty rows)
   while (lo < hi) {
@@ -243,7 +260,7 @@ __device__ __forceinline__ void decode_tile(const TileJob &J, int64_t idx, int &
   lr = lo;
   ti = J.orow[lo];
   tj = ti + (int)(idx - pre(lo));
-  if (ti < k && tj >= k) ++tj;
+  if (ti < k && tj >= k) tj += rest ? 2 : 1;
 }
 
 template <class CF>
@@ -612,26 +629,29 @@ struct TileJob16 {
   int32_t nown, mk, posk;
   unsigned long long *dbg;   // development (EAR_FW16_DBG): per-CTA %globaltimer at start / end, or null
   int32_t ti0;               // first tile row held by C (MODE_PIVOT_ROW on a standalone pivot row block: k)
+  int32_t posk1;             // MODE_LIST_CROSS / _REST
+  int32_t *counter;          // kDYN: {next tile, CTAs done}, zero at launch, reset by the last CTA
 };
 
 // LAR = 1: a ring stage is refilled by the LAST warp to finish consuming it (a shared counter) instead
 // of thread 0 waiting on an 'empty' barrier at the start of each chunk (which ties warp 0 to the
 // slowest warp every chunk).
-template <int KC, int STAGES, int MINB, int UNR, int NTH = 256, int PFC = 0, int LAR = 0, int SPIN = 0>
+template <int KC, int STAGES, int MINB, int UNR, int NTH = 256, int PFC = 0, int LAR = 0, int SPIN = 0,
+          int DYN = 0>
 struct Fw16Cfg {
   static constexpr int NCHUNK = TILE / KC;
   static constexpr int A_CHUNK = KC * TILE;   // u16 elements
   static constexpr int B_CHUNK = KC * TILE;   // u32 elements
-  static constexpr int SMEM = STAGES * (A_CHUNK * 2 + B_CHUNK * 4) + 2 * STAGES * 8 + STAGES * 4;
+  static constexpr int SMEM = STAGES * (A_CHUNK * 2 + B_CHUNK * 4) + 2 * STAGES * 8 + STAGES * 4 + 8;
   static constexpr int kKC = KC, kSTAGES = STAGES, kMINB = MINB, kUNR = UNR, kNTH = NTH, kPFC = PFC, kLAR = LAR;
-  static constexpr int kSPIN = SPIN;
+  static constexpr int kSPIN = SPIN, kDYN = DYN;
   static constexpr int RPH = 256 * 2 / NTH;   // row pairs per 64-row half owned by a thread (2 or 4)
 };
 
 __device__ __forceinline__ void decode16(const TileJob16 &J, int64_t idx, int &ti, int &tj, int &lr) {
   TileJob T{};
   T.k = J.k; T.nt = J.nt; T.mode = J.mode; T.ti0 = J.ti0;
-  T.orow = J.orow; T.opre = J.opre; T.nown = J.nown; T.mk = J.mk; T.posk = J.posk;
+  T.orow = J.orow; T.opre = J.opre; T.nown = J.nown; T.mk = J.mk; T.posk = J.posk; T.posk1 = J.posk1;
   decode_tile(T, idx, ti, tj, lr);
 }
 
@@ -814,6 +834,192 @@ __global__ void __launch_bounds__(CF::kNTH, CF::kMINB)
   }
 }
 
+// Dynamically scheduled version of k_fw_tiles16 (CF::kDYN): a CTA takes its next tile from a global
+// counter when it issues that tile's first TMA chunk, instead of the static blockIdx + it * grid
+// assignment.  Measured with the static assignment (tools/fw16_cta_times.py): all CTAs start
+// together but end between 43 % and 100 % of the launch -- the SM's warp scheduler favours its oldest
+// CTA, so the three CTAs of an SM run at different speeds and each SM spends the last part of every
+// launch with one or two of them (2.15 resident CTAs on average).  With the counter, fast CTAs simply
+// take more tiles.  The tile of a CTA's tile sequence number q is published in tslot[q & 1] (tagged
+// with q) by the thread that issues its first chunk; the ring depth (2) never exceeds the chunks per
+// tile (4), so a slot is rewritten only after every warp has read it.  The last CTA to finish resets
+// the counter pair for the next launch on the same stream.
+template <class CF>
+__global__ void __launch_bounds__(CF::kNTH, CF::kMINB)
+    k_fw_tiles16_dyn(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
+                     const TileJob16 J) {
+  constexpr int KC = CF::kKC, NCHUNK = CF::NCHUNK, STAGES = CF::kSTAGES, NTH = CF::kNTH, RPH = CF::RPH;
+  constexpr int NRP = 2 * RPH, NW = NTH / 32;
+  static_assert(NCHUNK >= STAGES, "tile slots are rewritten only after every warp has read them");
+  constexpr int32_t NONE = 0xFFFFF;
+  extern __shared__ __align__(128) uint8_t smem16[];
+  uint16_t *sA = reinterpret_cast<uint16_t *>(smem16);
+  uint32_t *sB = reinterpret_cast<uint32_t *>(sA + STAGES * CF::A_CHUNK);
+  uint64_t *full = reinterpret_cast<uint64_t *>(sB + STAGES * CF::B_CHUNK);
+  int32_t *cnt = reinterpret_cast<int32_t *>(full + 2 * STAGES);   // [STAGES] warps done with the stage
+  int32_t *tslot = cnt + STAGES;                                   // [2] (q << 20) | tile
+  const int tid = threadIdx.x, lane = tid & 31;
+  const int tx = tid & 15, ty = tid >> 4;
+  if (J.dbg && tid == 0) {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    uint32_t smid;
+    asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+    J.dbg[3 * blockIdx.x] = t;
+    J.dbg[3 * blockIdx.x + 2] = smid;
+  }
+  // chunk c of this CTA's sequence into stage st (one thread)
+  auto issue = [&](int c, int st) {
+    const int q = c / NCHUNK, kc = c % NCHUNK;
+    int32_t t;
+    if (kc == 0) {
+      const int32_t tt = atomicAdd(J.counter, 1);
+      t = tt < J.ntiles ? tt : -1;
+      tslot[q & 1] = (q << 20) | (t < 0 ? NONE : t);
+      __threadfence_block();
+    } else {
+      const int32_t v = tslot[q & 1] & NONE;
+      t = v == NONE ? -1 : v;
+    }
+    if (t < 0) {   // no tile: complete the phase without data so that the waiters see the end
+      mbar_arrive(&full[st]);
+      return;
+    }
+    int pti, ptj, plr;
+    decode16(J, t, pti, ptj, plr);
+    mbar_arrive_tx(&full[st], CF::A_CHUNK * 2 + CF::B_CHUNK * 4);
+    tma_load_2d(sA + st * CF::A_CHUNK, &tmA, pti * TILE, J.a_row0 + kc * KC, &full[st]);
+    tma_load_2d(sB + st * CF::B_CHUNK, &tmB, ptj * TILE, kc * KC, &full[st]);
+  };
+  if (tid == 0) {
+    for (int s = 0; s < STAGES; ++s) {
+      mbar_init(&full[s], 1);
+      cnt[s] = 0;
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
+    asm volatile("prefetch.tensormap [%0];\n" ::"l"(reinterpret_cast<uint64_t>(&tmA)) : "memory");
+    asm volatile("prefetch.tensormap [%0];\n" ::"l"(reinterpret_cast<uint64_t>(&tmB)) : "memory");
+  }
+  __syncthreads();
+  if (tid == 0)
+    for (int c = 0; c < STAGES; ++c) issue(c, c);
+
+  auto row_of = [&](int r2) { return (r2 < RPH ? 0 : 64) + ty * 2 * RPH + (r2 % RPH) * 2; };
+  int g = 0;
+  for (int q = 0;; ++q) {
+    mbar_wait(&full[g % STAGES], (uint32_t)((g / STAGES) & 1));
+    const int32_t v = tslot[q & 1] & NONE;
+    if (v == NONE) break;
+    int ti, tj, lr;
+    decode16(J, v, ti, tj, lr);
+    uint32_t c[NRP][8];
+    uint16_t *Ct = J.C + (int64_t)lr * TILE * J.ldc + (int64_t)tj * TILE;
+#pragma unroll
+    for (int r2 = 0; r2 < NRP; ++r2) {
+      const int i = row_of(r2);
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        const uint2 a = *reinterpret_cast<const uint2 *>(Ct + (int64_t)i * J.ldc + h * 64 + tx * 4);
+        const uint2 b = *reinterpret_cast<const uint2 *>(Ct + (int64_t)(i + 1) * J.ldc + h * 64 + tx * 4);
+        c[r2][h * 4 + 0] = __byte_perm(a.x, b.x, 0x5410);
+        c[r2][h * 4 + 1] = __byte_perm(a.x, b.x, 0x7632);
+        c[r2][h * 4 + 2] = __byte_perm(a.y, b.y, 0x5410);
+        c[r2][h * 4 + 3] = __byte_perm(a.y, b.y, 0x7632);
+      }
+    }
+#pragma unroll 1
+    for (int kc = 0; kc < NCHUNK; ++kc, ++g) {
+      const int st = g % STAGES;
+      if (kc > 0) mbar_wait(&full[st], (uint32_t)((g / STAGES) & 1));
+      if (CF::kPFC && kc == NCHUNK - 1) {   // the next tile, once published: its C rows into L2
+        const int32_t nv = tslot[(q + 1) & 1];
+        if ((nv >> 20) == q + 1 && (nv & NONE) != NONE) {
+          int nti, ntj, nlr;
+          decode16(J, nv & NONE, nti, ntj, nlr);
+          const uint16_t *Cn = J.C + (int64_t)nlr * TILE * J.ldc + (int64_t)ntj * TILE;
+          for (int l = tid; l < 2 * TILE; l += NTH)
+            asm volatile("prefetch.global.L2::evict_last [%0];" ::"l"(Cn + (int64_t)(l >> 1) * J.ldc + (l & 1) * 64));
+        }
+      }
+      const uint16_t *a_s = sA + st * CF::A_CHUNK;
+      const uint32_t *b_s = sB + st * CF::B_CHUNK;
+#pragma unroll CF::kUNR
+      for (int kk = 0; kk < KC; ++kk) {
+        uint32_t a[NRP];
+        if (RPH == 2) {
+          const uint2 alo = *reinterpret_cast<const uint2 *>(a_s + kk * TILE + ty * 4);
+          const uint2 ahi = *reinterpret_cast<const uint2 *>(a_s + kk * TILE + 64 + ty * 4);
+          a[0] = alo.x; a[1] = alo.y; a[RPH] = ahi.x; a[RPH + 1] = ahi.y;
+        } else {
+          const uint4 alo = *reinterpret_cast<const uint4 *>(a_s + kk * TILE + ty * 8);
+          const uint4 ahi = *reinterpret_cast<const uint4 *>(a_s + kk * TILE + 64 + ty * 8);
+          a[0] = alo.x; a[1] = alo.y; a[2] = alo.z; a[3] = alo.w;
+          a[RPH] = ahi.x; a[RPH + 1] = ahi.y; a[RPH + 2] = ahi.z; a[RPH + 3] = ahi.w;
+        }
+        const uint4 blo = *reinterpret_cast<const uint4 *>(b_s + kk * TILE + tx * 4);
+        const uint4 bhi = *reinterpret_cast<const uint4 *>(b_s + kk * TILE + 64 + tx * 4);
+        const uint32_t b[8] = {blo.x, blo.y, blo.z, blo.w, bhi.x, bhi.y, bhi.z, bhi.w};
+#pragma unroll
+        for (int r2 = 0; r2 < NRP; ++r2)
+#pragma unroll
+          for (int qq = 0; qq < 8; ++qq) c[r2][qq] = __viaddmin_u16x2(a[r2], b[qq], c[r2][qq]);
+      }
+      __syncwarp();
+      if (lane == 0) {
+        __threadfence_block();
+        if (atomicAdd(&cnt[st], 1) == NW - 1) {   // the last reader of this stage refills it
+          cnt[st] = 0;
+          __threadfence_block();
+          asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");
+          issue(g + STAGES, st);
+        }
+      }
+    }
+#pragma unroll
+    for (int r2 = 0; r2 < NRP; ++r2) {
+      const int i = row_of(r2);
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        const uint32_t *cc = &c[r2][h * 4];
+        *reinterpret_cast<uint2 *>(Ct + (int64_t)i * J.ldc + h * 64 + tx * 4) =
+            make_uint2(__byte_perm(cc[0], cc[1], 0x5410), __byte_perm(cc[2], cc[3], 0x5410));
+        *reinterpret_cast<uint2 *>(Ct + (int64_t)(i + 1) * J.ldc + h * 64 + tx * 4) =
+            make_uint2(__byte_perm(cc[0], cc[1], 0x7632), __byte_perm(cc[2], cc[3], 0x7632));
+      }
+    }
+    if (J.mirror && ti != tj) {
+      uint16_t *Mt = J.C + (int64_t)tj * TILE * J.ldc + (int64_t)ti * TILE;
+#pragma unroll
+      for (int qq = 0; qq < 8; ++qq) {
+        const int j = (qq < 4 ? 0 : 64) + tx * 4 + (qq & 3);
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+          if (RPH == 2) {
+            *reinterpret_cast<uint2 *>(Mt + (int64_t)j * J.ldc + h * 64 + ty * 4) = make_uint2(c[h * 2][qq], c[h * 2 + 1][qq]);
+          } else {
+            *reinterpret_cast<uint4 *>(Mt + (int64_t)j * J.ldc + h * 64 + ty * 8) =
+                make_uint4(c[h * 4][qq], c[h * 4 + 1][qq], c[h * 4 + 2][qq], c[h * 4 + 3][qq]);
+          }
+        }
+      }
+    }
+  }
+  __syncthreads();
+  if (tid == 0) {
+    if (J.dbg) {
+      unsigned long long t;
+      asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+      J.dbg[3 * blockIdx.x + 1] = t;
+    }
+    __threadfence();
+    if (atomicAdd(J.counter + 1, 1) == (int)gridDim.x - 1) {   // the last CTA resets the pair
+      J.counter[0] = 0;
+      J.counter[1] = 0;
+      __threadfence();
+    }
+  }
+}
+
 // connected-component labels (min vertex id) of the reduced graph by hooking + pointer jumping
 __global__ void k_cc_init(int32_t *lab, int32_t n) {
   for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x)
@@ -908,34 +1114,62 @@ ear_status_t launch_tiles(const CUtensorMap &map, TileJob J, int64_t nblocks, cu
 // variants, profiles/r01_fw16_variants.jsonl): 128 threads with 16 x 8 values each, 32-deep k-chunks,
 // a 2-stage TMA ring (48 KB), 3 CTAs per SM, kk unrolled 16x; then (tools/lab_fw16_variant.sh,
 // profiles/r01u_fw16_refill.jsonl) last-arriver refills of the ring and an L2 prefetch of the next
-// C tile: 475.3 -> 471.6 ms on cfg4's plain FW (3-stage rings and 16-deep chunks measured slower).
-using Fw16Tile = Fw16Cfg<32, 2, 3, 16, 128, 1, 1>;
+// C tile: 475.3 -> 471.6 ms on cfg4's plain FW (3-stage rings and 16-deep chunks measured slower);
+// then dynamic tile scheduling (k_fw_tiles16_dyn, the CTAs of an SM run at different speeds) and 4 CTA
+// slots left to the lookahead's pivot chain: 472.7 -> 445.9 ms (profiles/r01y_fw16_dyn.jsonl).
+using Fw16Tile = Fw16Cfg<32, 2, 3, 16, 128, 0, 1, 0, 1>;   // dynamic tile scheduling (k_fw_tiles16_dyn)
 using Fw16TileL = Fw16Cfg<32, 2, 3, 16, 128, 0, 1>;
 using Fw16TileL4 = Fw16Cfg<16, 4, 3, 16, 128, 0, 1>;
 using Fw16TileL3 = Fw16Cfg<32, 3, 3, 16, 128, 0, 1>;
-using Fw16TileLP = Fw16Cfg<32, 2, 3, 16, 128, 1, 1>;
+using Fw16TileLP = Fw16Cfg<32, 2, 3, 16, 128, 1, 1>;   // the static default before the tile counter
 using Fw16TileL3P = Fw16Cfg<32, 3, 3, 16, 128, 1, 1>;
 using Fw16TileS = Fw16Cfg<32, 2, 3, 16, 128, 1, 1, 1>;
 using Fw16TileS3 = Fw16Cfg<32, 3, 3, 16, 128, 1, 1, 1>;
+using Fw16TileD = Fw16Cfg<32, 2, 3, 16, 128, 1, 1, 0, 1>;
+using Fw16TileD0 = Fw16Cfg<32, 2, 3, 16, 128, 0, 1, 0, 1>;
 
 // development knobs (tools/): EAR_FW16_LOOKAHEAD=0 disables the lookahead, EAR_FW16_RESERVE sets the
-// CTA slots the rest-of-round launch leaves free for the next round's pivot work (default 0: measured
-// best, profiles/r01_fw16_lookahead.jsonl), EAR_FW16_PRIO=0 gives the side stream normal priority
+// CTA slots the rest-of-round launch leaves free for the next round's pivot work (default 4: with the
+// persistent dynamically scheduled kernel no slot frees up before the launch drains; measured best,
+// profiles/r01y_fw16_dyn.jsonl), EAR_FW16_PRIO=0 gives the side stream normal priority
 int env_int(const char *name, int dflt) {
   const char *e = getenv(name);
   return e ? atoi(e) : dflt;
 }
 
+// the dynamic kernel's counter pair for launches on stream st: one pair per (device, stream), zeroed
+// once and reset by each launch's last CTA, so launches on one stream reuse it in order
+int32_t *dyn_counter(cudaStream_t st) {
+  static std::vector<std::pair<std::pair<int, cudaStream_t>, int32_t *>> pairs;
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess) return nullptr;
+  for (auto &p : pairs)
+    if (p.first.first == dev && p.first.second == st) return p.second;
+  int32_t *c = nullptr;
+  if (cudaMalloc((void **)&c, 2 * sizeof(int32_t)) != cudaSuccess || cudaMemset(c, 0, 2 * sizeof(int32_t)) != cudaSuccess)
+    return nullptr;
+  pairs.push_back({{dev, st}, c});
+  return c;
+}
+
 template <class CF>
 ear_status_t launch16_cfg(const CUtensorMap &mA, const CUtensorMap &mB, TileJob16 J, int64_t nblocks, cudaStream_t st,
                           int reserve) {
+  auto kern = CF::kDYN ? k_fw_tiles16_dyn<CF> : k_fw_tiles16<CF>;
   static bool attr = false;
   if (!attr) {
-    EAR_CUDA_TRY(cudaFuncSetAttribute(k_fw_tiles16<CF>, cudaFuncAttributeMaxDynamicSharedMemorySize, CF::SMEM));
+    EAR_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, CF::SMEM));
     attr = true;
   }
+  if (CF::kDYN) {
+    J.counter = dyn_counter(st);
+    if (!J.counter) {
+      set_error("fw16: no tile counter");
+      return EAR_ECUDA;
+    }
+  }
   int per_sm = 0;
-  EAR_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_fw_tiles16<CF>, CF::kNTH, CF::SMEM));
+  EAR_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, CF::kNTH, CF::SMEM));
   if (per_sm < 1) per_sm = 1;
   J.ntiles = nblocks;
   const int64_t grid = std::min<int64_t>(nblocks, std::max<int64_t>(1, (int64_t)g_num_sms * per_sm - reserve));
@@ -944,7 +1178,7 @@ ear_status_t launch16_cfg(const CUtensorMap &mA, const CUtensorMap &mB, TileJob1
   static int nlaunch = 0;
   const bool dbg = dbg_at >= 0 && nlaunch++ == dbg_at;
   if (dbg) EAR_CUDA_TRY(cudaMalloc((void **)&J.dbg, sizeof(unsigned long long) * 3 * grid));
-  EAR_LAUNCH(k_fw_tiles16<CF>, (unsigned)grid, CF::kNTH, CF::SMEM, st)(mA, mB, J);
+  EAR_LAUNCH(kern, (unsigned)grid, CF::kNTH, CF::SMEM, st)(mA, mB, J);
   if (dbg) {
     std::vector<unsigned long long> h(3 * grid);
     EAR_CUDA_TRY(cudaStreamSynchronize(st));
@@ -961,8 +1195,9 @@ ear_status_t launch16_cfg(const CUtensorMap &mA, const CUtensorMap &mB, TileJob1
 
 int fw16_kc() { return env_int("EAR_FW16_VARIANT", 0) == 2 ? Fw16TileL4::kKC : Fw16Tile::kKC; }
 
-// EAR_FW16_VARIANT (development knob, tools/lab_fw16_variant.sh): 0 = Fw16Tile, 1 = last-arriver refill
-// without the C prefetch, 2 = 4-stage ring of 16-deep chunks, 3 = 3-stage ring, 5 = 3-stage + prefetch
+// EAR_FW16_VARIANT (development knob, tools/lab_fw16_*.sh): 0 = Fw16Tile; static tile assignment:
+// 1 = last-arriver refill, 2 = 4-stage ring of 16-deep chunks, 3 = 3-stage ring, 4 = refill + C prefetch
+// (the static default before), 5 = 3-stage + prefetch, 6/7 = polling waits; 8 = dynamic + C prefetch
 template <class CF>
 ear_status_t launch16(const CUtensorMap &mA, const CUtensorMap &mB, TileJob16 J, int64_t nblocks, cudaStream_t st,
                       int reserve = 0) {
@@ -975,10 +1210,33 @@ ear_status_t launch16(const CUtensorMap &mA, const CUtensorMap &mB, TileJob16 J,
   if (variant == 5) return launch16_cfg<Fw16TileL3P>(mA, mB, J, nblocks, st, reserve);
   if (variant == 6) return launch16_cfg<Fw16TileS>(mA, mB, J, nblocks, st, reserve);
   if (variant == 7) return launch16_cfg<Fw16TileS3>(mA, mB, J, nblocks, st, reserve);
+  if (variant == 8) return launch16_cfg<Fw16TileD>(mA, mB, J, nblocks, st, reserve);
+  if (variant == 9) return launch16_cfg<Fw16TileD0>(mA, mB, J, nblocks, st, reserve);
   return launch16_cfg<CF>(mA, mB, J, nblocks, st, reserve);
 }
 
 int grid_for(int64_t n) { return (int)std::max<int64_t>(1, std::min<int64_t>(ceil_div(n, 256), 148 * 16)); }
+
+// the lookahead's side stream and events of the current device (created once, shared by the single-GPU
+// and the sharded packed FW; one FW call at a time per device)
+ear_status_t side_stream(cudaStream_t *side, cudaEvent_t *ev_cross, cudaEvent_t *ev_pivot) {
+  static cudaStream_t sides[64] = {};
+  static cudaEvent_t crosses[64] = {}, pivots[64] = {};
+  int dev = 0;
+  EAR_CUDA_TRY(cudaGetDevice(&dev));
+  if (dev < 0 || dev >= 64) { set_error("side_stream: device %d out of range", dev); return EAR_EINVAL; }
+  if (!sides[dev]) {
+    int lo = 0, hi = 0;   // the pivot work gets the highest priority: its CTAs take the first free slots
+    EAR_CUDA_TRY(cudaDeviceGetStreamPriorityRange(&lo, &hi));
+    EAR_CUDA_TRY(cudaStreamCreateWithPriority(&sides[dev], cudaStreamNonBlocking, env_int("EAR_FW16_PRIO", 1) ? hi : lo));
+    EAR_CUDA_TRY(cudaEventCreateWithFlags(&crosses[dev], cudaEventDisableTiming));
+    EAR_CUDA_TRY(cudaEventCreateWithFlags(&pivots[dev], cudaEventDisableTiming));
+  }
+  *side = sides[dev];
+  *ev_cross = crosses[dev];
+  *ev_pivot = pivots[dev];
+  return EAR_OK;
+}
 
 // The packed 16-bit FW on a copy of D (see C16 above).  *done = false (D untouched) when a connected
 // pair reached the cap; the caller then runs the int32 FW.  Synchronises the stream once (the check).
@@ -997,23 +1255,11 @@ ear_status_t fw_single16(int32_t *D, int64_t ldd, int32_t Np, const int32_t *lab
     EAR_CUDA_TRY(cudaGetDevice(&dev));
     EAR_CUDA_TRY(cudaDeviceGetAttribute(&g_num_sms, cudaDevAttrMultiProcessorCount, dev));
   }
-  // per-device side stream and the two lookahead events (created once)
-  static cudaStream_t sides[64] = {};
-  static cudaEvent_t crosses[64] = {}, pivots[64] = {};
-  int dev = 0;
-  EAR_CUDA_TRY(cudaGetDevice(&dev));
-  if (dev < 0 || dev >= 64) { set_error("fw_single16: device %d out of range", dev); return EAR_EINVAL; }
-  if (!sides[dev]) {
-    int lo = 0, hi = 0;   // the pivot work gets the highest priority: its CTAs take the first free slots
-    EAR_CUDA_TRY(cudaDeviceGetStreamPriorityRange(&lo, &hi));
-    EAR_CUDA_TRY(cudaStreamCreateWithPriority(&sides[dev], cudaStreamNonBlocking, env_int("EAR_FW16_PRIO", 1) ? hi : lo));
-    EAR_CUDA_TRY(cudaEventCreateWithFlags(&crosses[dev], cudaEventDisableTiming));
-    EAR_CUDA_TRY(cudaEventCreateWithFlags(&pivots[dev], cudaEventDisableTiming));
-  }
-  cudaStream_t side = sides[dev];
-  cudaEvent_t ev_cross = crosses[dev], ev_pivot = pivots[dev];
+  cudaStream_t side;
+  cudaEvent_t ev_cross, ev_pivot;
+  EAR_TRY(side_stream(&side, &ev_cross, &ev_pivot));
   const bool lookahead = env_int("EAR_FW16_LOOKAHEAD", 1) != 0;
-  const int reserve = env_int("EAR_FW16_RESERVE", 0);
+  const int reserve = env_int("EAR_FW16_RESERVE", 4);
   const int nt = Np / TILE;
   const double tile_ops = (double)TILE * TILE * TILE;
   uint16_t *D16 = nullptr;
@@ -1320,22 +1566,36 @@ ear_status_t fw_sharded(int32_t *S, int64_t ldd, int32_t Np, ear_comm_s *comm, c
 // disjoint, so no exchange is needed).  The range check runs over every rank's owned upper tiles and
 // is MIN-reduced; *done = false leaves the int32 owned storage untouched for the int32 schedule.
 static ear_status_t phase3_16(const Shard &sh, uint16_t *S16, const CUtensorMap &mA, const CUtensorMap &mB, int k,
-                              cudaStream_t st) {
-  int mk = 0, posk = -1;
+                              int mode, cudaStream_t st, int reserve = 0) {
+  int mk = 0, posk = -1, posk1 = -1;
   int64_t total = 0;
   for (int32_t r = 0; r < sh.nown; ++r) {
     const int32_t ti = sh.rows[r];
     if (ti < k) ++mk;
     if (ti == k) posk = r;
-    total += ti == k ? 0 : (sh.nt - ti) - (ti < k ? 1 : 0);
+    if (ti == k + 1) posk1 = r;
   }
-  TileJob16 J{S16, sh.Np, 0, k, sh.nt, MODE_LIST, 0, 0, sh.d_rows, sh.d_pre, sh.nown, mk, posk};
+  for (int32_t r = 0; r < sh.nown; ++r) {
+    const int32_t ti = sh.rows[r];
+    const int64_t all = ti == k ? 0 : (sh.nt - ti) - (ti < k ? 1 : 0);
+    const int64_t cross = (ti == k + 1 ? sh.nt - ti : 0) + (ti < k ? 1 : 0);
+    total += mode == MODE_LIST ? all : mode == MODE_LIST_CROSS ? cross : all - cross;
+  }
+  if (total == 0) return EAR_OK;
+  TileJob16 J{S16, sh.Np, 0, k, sh.nt, mode, 0, 0, sh.d_rows, sh.d_pre, sh.nown, mk, posk};
+  J.posk1 = posk1;
   int s3 = prof_begin(PK_FW_P3_16, st);
-  EAR_TRY(launch16<Fw16Tile>(mA, mB, J, total, st));
+  EAR_TRY(launch16<Fw16Tile>(mA, mB, J, total, st, reserve));
   prof_end(s3, st, (double)total * TILE * TILE * TILE);
   return EAR_OK;
 }
 
+// Lookahead (as fw_single16's): round k's phase 3 is split into the owned tiles of row/column k+1
+// (MODE_LIST_CROSS, first) and the rest (MODE_LIST_REST); once the cross tiles are done, round k+1's
+// pivot chain -- pieces into the exchange block, the all-reduce, narrowing, phases 1-2, scatter back --
+// runs on the side stream (NCCL included) while the rest of round k proceeds; the two touch disjoint
+// tiles, the narrowed block and its duplicate alternate between two buffers by round parity, and round
+// k+1's phase 3 waits for the chain.
 static ear_status_t fw_sharded16(std::vector<Shard *> &sh, int32_t Np, ear_comm_s *comm, const int32_t *lab,
                                  int32_t n_real, bool *done, cudaStream_t st, bool timing_only = false) {
   *done = false;
@@ -1346,14 +1606,19 @@ static ear_status_t fw_sharded16(std::vector<Shard *> &sh, int32_t Np, ear_comm_
     EAR_CUDA_TRY(cudaGetDevice(&dev));
     EAR_CUDA_TRY(cudaDeviceGetAttribute(&g_num_sms, cudaDevAttrMultiProcessorCount, dev));
   }
+  cudaStream_t side;
+  cudaEvent_t ev_cross, ev_pivot;
+  EAR_TRY(side_stream(&side, &ev_cross, &ev_pivot));
+  const bool lookahead = env_int("EAR_FW16_LOOKAHEAD", 1) != 0;
+  const int reserve = env_int("EAR_FW16_RESERVE", 4);
   const size_t R = sh.size();
   std::vector<uint16_t *> S16(R, nullptr);
   int32_t *prow = nullptr, *flag = nullptr;
-  uint16_t *p16 = nullptr;
+  uint16_t *p16 = nullptr;   // two 128 x Np buffers (round parity), as Pd
   uint32_t *Pd = nullptr;
   bool ok = cudaMallocAsync((void **)&prow, sizeof(int32_t) * (size_t)TILE * Np, st) == cudaSuccess &&
-            cudaMallocAsync((void **)&p16, sizeof(uint16_t) * (size_t)TILE * Np, st) == cudaSuccess &&
-            cudaMallocAsync((void **)&Pd, sizeof(uint32_t) * (size_t)TILE * Np, st) == cudaSuccess &&
+            cudaMallocAsync((void **)&p16, 2 * sizeof(uint16_t) * (size_t)TILE * Np, st) == cudaSuccess &&
+            cudaMallocAsync((void **)&Pd, 2 * sizeof(uint32_t) * (size_t)TILE * Np, st) == cudaSuccess &&
             cudaMallocAsync((void **)&flag, sizeof(int32_t), st) == cudaSuccess;
   for (size_t r = 0; r < R && ok; ++r)
     ok = cudaMallocAsync((void **)&S16[r], sizeof(uint16_t) * (size_t)std::max(sh[r]->nown, 1) * TILE * Np, st) ==
@@ -1373,9 +1638,12 @@ static ear_status_t fw_sharded16(std::vector<Shard *> &sh, int32_t Np, ear_comm_
   }
   const int KC = fw16_kc();
   const int64_t nblk = (int64_t)TILE * Np;
-  CUtensorMap mA, mB;
-  ear_status_t s = make_map_t(&mA, CU_TENSOR_MAP_DATA_TYPE_UINT16, 2, p16, TILE, Np, Np, KC);
-  if (s == EAR_OK) s = make_map_t(&mB, CU_TENSOR_MAP_DATA_TYPE_UINT32, 4, Pd, TILE, Np, Np, KC);
+  CUtensorMap mA[2], mB[2];
+  ear_status_t s = EAR_OK;
+  for (int b = 0; b < 2 && s == EAR_OK; ++b) {
+    s = make_map_t(&mA[b], CU_TENSOR_MAP_DATA_TYPE_UINT16, 2, p16 + b * nblk, TILE, Np, Np, KC);
+    if (s == EAR_OK) s = make_map_t(&mB[b], CU_TENSOR_MAP_DATA_TYPE_UINT32, 4, Pd + b * nblk, TILE, Np, Np, KC);
+  }
   if (s == EAR_OK) {
     int sc = prof_begin(PK_FW16_CONV, st);
     for (size_t r = 0; r < R; ++r)
@@ -1384,35 +1652,55 @@ static ear_status_t fw_sharded16(std::vector<Shard *> &sh, int32_t Np, ear_comm_
             sh[r]->S, sh[r]->ldd, S16[r], Np, (int64_t)sh[r]->nown * TILE, Np);
     prof_end(sc, st, 0);
   }
-  for (int k = 0; k < nt && s == EAR_OK; ++k) {
-    s = fill(prow, nblk, INF, st);
-    for (size_t r = 0; r < R && s == EAR_OK; ++r)
-      if (sh[r]->nown > 0)
-        s = shard_xfer_t<uint16_t, int32_t>(*sh[r], S16[r], Np, k, prow, 0, st);
-    if (s == EAR_OK && comm) {
-      int sc = prof_begin(PK_COMM, st);
-      s = comm_allreduce_min(comm, prow, nblk, st);
-      prof_end(sc, st, 0);
-    }
-    if (s != EAR_OK) break;
-    // phases 1-2 packed, as fw_single16's pivot(): narrow, close the pivot tile, B = the pre-phase-2
-    // row duplicated, the pivot-row tiles as one product, then B again for phase 3
-    EAR_LAUNCH(k_prow_to16, grid_for(nblk / 4), 256, 0, st)(prow, p16, nullptr, nblk);
-    int s1 = prof_begin(PK_FW_P1, st);
-    EAR_LAUNCH(k_fw_phase1_16, 1, NT, 0, st)(p16 + (int64_t)k * TILE, Np);
-    prof_end(s1, st, (double)TILE * TILE * TILE);
-    int s2 = prof_begin(PK_FW_P2, st);
-    EAR_LAUNCH(k_dup16, grid_for(nblk / 4), 256, 0, st)(p16, Np, Pd);
-    TileJob16 J2{p16, Np, 0, k, nt, MODE_PIVOT_ROW, 0, 0};
-    J2.ti0 = k;
-    s = launch16<Fw16Tile>(mA, mB, J2, nt - 1, st);
-    EAR_LAUNCH(k_dup16, grid_for(nblk / 4), 256, 0, st)(p16, Np, Pd);
-    prof_end(s2, st, (double)(nt - 1) * TILE * TILE * TILE);
-    if (s != EAR_OK) break;
+  // round k's pivot chain on stream q: pieces -> exchange -> narrowed block (buffer k & 1) -> phases
+  // 1-2 packed, as fw_single16's pivot() -> scattered back to the owners
+  auto chain = [&](int k, cudaStream_t q) -> ear_status_t {
+    const bool on_side = q != st;
+    uint16_t *P16 = p16 + (k & 1) * nblk;
+    uint32_t *Pk = Pd + (k & 1) * nblk;
+    EAR_TRY(fill(prow, nblk, INF, q));
     for (size_t r = 0; r < R; ++r)
-      if (sh[r]->nown > 0)
-        s = shard_xfer_t<uint16_t, uint16_t>(*sh[r], S16[r], Np, k, p16, 1, st);
-    for (size_t r = 0; r < R && s == EAR_OK; ++r) s = phase3_16(*sh[r], S16[r], mA, mB, k, st);
+      if (sh[r]->nown > 0) EAR_TRY((shard_xfer_t<uint16_t, int32_t>(*sh[r], S16[r], Np, k, prow, 0, q)));
+    if (comm) {
+      int sc = prof_begin(PK_COMM, q);
+      EAR_TRY(comm_allreduce_min(comm, prow, nblk, q));
+      prof_end(sc, q, 0);
+    }
+    EAR_LAUNCH(k_prow_to16, grid_for(nblk / 4), 256, 0, q)(prow, P16, nullptr, nblk);
+    int s1 = prof_begin(on_side ? PK_FW_SIDE_P1 : PK_FW_P1, q);
+    EAR_LAUNCH(k_fw_phase1_16, 1, NT, 0, q)(P16 + (int64_t)k * TILE, Np);
+    prof_end(s1, q, (double)TILE * TILE * TILE);
+    int s2 = prof_begin(on_side ? PK_FW_SIDE_P2 : PK_FW_P2, q);
+    EAR_LAUNCH(k_dup16, grid_for(nblk / 4), 256, 0, q)(P16, Np, Pk);
+    TileJob16 J2{P16, Np, 0, k, nt, MODE_PIVOT_ROW, 0, 0};
+    J2.ti0 = k;
+    EAR_TRY(launch16<Fw16Tile>(mA[k & 1], mB[k & 1], J2, nt - 1, q));
+    EAR_LAUNCH(k_dup16, grid_for(nblk / 4), 256, 0, q)(P16, Np, Pk);
+    prof_end(s2, q, (double)(nt - 1) * TILE * TILE * TILE);
+    for (size_t r = 0; r < R; ++r)
+      if (sh[r]->nown > 0) EAR_TRY((shard_xfer_t<uint16_t, uint16_t>(*sh[r], S16[r], Np, k, P16, 1, q)));
+    return EAR_OK;
+  };
+  if (s == EAR_OK) s = chain(0, st);
+  for (int k = 0; k < nt && s == EAR_OK; ++k) {
+    const CUtensorMap &A = mA[k & 1], &B = mB[k & 1];
+    if (!lookahead || k + 1 == nt) {
+      for (size_t r = 0; r < R && s == EAR_OK; ++r) s = phase3_16(*sh[r], S16[r], A, B, k, MODE_LIST, st);
+      if (s == EAR_OK && k + 1 < nt) s = chain(k + 1, st);
+      continue;
+    }
+    for (size_t r = 0; r < R && s == EAR_OK; ++r) s = phase3_16(*sh[r], S16[r], A, B, k, MODE_LIST_CROSS, st);
+    if (s != EAR_OK) break;
+    cudaError_t e = cudaEventRecord(ev_cross, st);
+    if (e == cudaSuccess) e = cudaStreamWaitEvent(side, ev_cross, 0);
+    if (e != cudaSuccess) { set_error("fw_sharded16: %s", cudaGetErrorString(e)); s = EAR_ECUDA; break; }
+    s = chain(k + 1, side);
+    e = cudaEventRecord(ev_pivot, side);   // recorded even after an error: the main stream waits for it
+    if (s == EAR_OK && e != cudaSuccess) { set_error("fw_sharded16: %s", cudaGetErrorString(e)); s = EAR_ECUDA; }
+    for (size_t r = 0; r < R && s == EAR_OK; ++r)
+      s = phase3_16(*sh[r], S16[r], A, B, k, MODE_LIST_REST, st, reserve);
+    e = cudaStreamWaitEvent(st, ev_pivot, 0);
+    if (s == EAR_OK && e != cudaSuccess) { set_error("fw_sharded16: %s", cudaGetErrorString(e)); s = EAR_ECUDA; }
   }
   int32_t h_flag = -1;
   if (s == EAR_OK && timing_only) {   // apsp_reduced_rank_timing: no check, no result

@@ -201,3 +201,15 @@ def test_sharded16_corner_equals_fw32(pkg, seed):
     assert p32["fw16_used"] == 0 and p32["fw16_fallbacks"] == 0
     assert np.array_equal(d16, d32)
     assert_exact(d16, oracle_on_terminals(g), f"sharded16 corner seed {seed}")
+
+
+@pytest.mark.parametrize("P", [1, 3, 8])
+def test_sharded16_without_lookahead(pkg, P, monkeypatch):
+    """The sharded packed schedule with its lookahead off (serial pivot chains) gives the same D."""
+    g = gg.corner_cases(4200 + P, n_target=1400)
+    d_la, _ = emulated(pkg, g, P)
+    monkeypatch.setenv("EAR_FW16_LOOKAHEAD", "0")
+    d_serial, prof = emulated(pkg, g, P)
+    assert prof["fw16_used"] == 1
+    assert np.array_equal(d_la, d_serial)
+    assert_exact(d_serial, oracle_on_terminals(g), f"sharded16 serial P={P}")
