@@ -244,7 +244,7 @@ def run_ours(args, rank, world, local_rank):
     bcc = None
     if args.phase2 == "bcc":
         pb = ea.ear_decompose(g.n, src, dst, w, flags=flags)
-        if world == 1:   # one untimed Phase II so that the re-reduction counts are those of a solve
+        if world == 1 and not args.no_alt:   # one untimed Phase II: the re-reduction counts of a solve
             Dp = ea.alloc_D(pb)
             ea.apsp_reduced(pb, Dp)
             torch.cuda.synchronize()

@@ -1217,6 +1217,20 @@ ear_status_t launch16(const CUtensorMap &mA, const CUtensorMap &mB, TileJob16 J,
 
 int grid_for(int64_t n) { return (int)std::max<int64_t>(1, std::min<int64_t>(ceil_div(n, 256), 148 * 16)); }
 
+// CTA slots the rest-of-round launch leaves to the next round's pivot chain.  The persistent,
+// dynamically scheduled tile kernel frees no slot before it drains, so the chain's phase-2 tiles (one
+// pivot row, p2 tiles) run on the reserved slots alongside the rest (rest tiles): enough slots that
+// they finish no later, p2 / R <= rest / (slots - R), plus one for phase 1.  EAR_FW16_RESERVE
+// overrides (measured on cfg4's single-GPU FW: 4 best, profiles/r01y_fw16_dyn.jsonl -- this rule
+// gives 5-6 there and ~28 at 8 ranks, where a rank's rest is 8x smaller).
+int lookahead_reserve(int64_t rest, int64_t p2) {
+  const int forced = env_int("EAR_FW16_RESERVE", -1);
+  if (forced >= 0) return forced;
+  const int64_t slots = (int64_t)std::max(g_num_sms, 1) * 3;
+  const int64_t r = (slots * p2 + rest + p2 - 1) / std::max<int64_t>(rest + p2, 1) + 1;
+  return (int)std::min<int64_t>(std::max<int64_t>(r, 1), slots / 2);
+}
+
 // the lookahead's side stream and events of the current device (created once, shared by the single-GPU
 // and the sharded packed FW; one FW call at a time per device)
 ear_status_t side_stream(cudaStream_t *side, cudaEvent_t *ev_cross, cudaEvent_t *ev_pivot) {
@@ -1259,7 +1273,6 @@ ear_status_t fw_single16(int32_t *D, int64_t ldd, int32_t Np, const int32_t *lab
   cudaEvent_t ev_cross, ev_pivot;
   EAR_TRY(side_stream(&side, &ev_cross, &ev_pivot));
   const bool lookahead = env_int("EAR_FW16_LOOKAHEAD", 1) != 0;
-  const int reserve = env_int("EAR_FW16_RESERVE", 4);
   const int nt = Np / TILE;
   const double tile_ops = (double)TILE * TILE * TILE;
   uint16_t *D16 = nullptr;
@@ -1327,7 +1340,7 @@ ear_status_t fw_single16(int32_t *D, int64_t ldd, int32_t Np, const int32_t *lab
     J.mode = MODE_REST;
     const int64_t nrest = (int64_t)(nt - 2) * (nt - 1) / 2;
     int s4 = prof_begin(PK_FW_P3_16, st);
-    s = launch16<Fw16Tile>(mA, mB[k & 1], J, nrest, st, reserve);
+    s = launch16<Fw16Tile>(mA, mB[k & 1], J, nrest, st, lookahead_reserve(nrest, nt - 1));
     prof_end(s4, st, nrest * tile_ops);
     if (s == EAR_OK) {
       e = cudaStreamWaitEvent(st, ev_pivot, 0);
@@ -1566,7 +1579,7 @@ ear_status_t fw_sharded(int32_t *S, int64_t ldd, int32_t Np, ear_comm_s *comm, c
 // disjoint, so no exchange is needed).  The range check runs over every rank's owned upper tiles and
 // is MIN-reduced; *done = false leaves the int32 owned storage untouched for the int32 schedule.
 static ear_status_t phase3_16(const Shard &sh, uint16_t *S16, const CUtensorMap &mA, const CUtensorMap &mB, int k,
-                              int mode, cudaStream_t st, int reserve = 0) {
+                              int mode, cudaStream_t st, int reserve = 0) {   // reserve < 0: lookahead_reserve
   int mk = 0, posk = -1, posk1 = -1;
   int64_t total = 0;
   for (int32_t r = 0; r < sh.nown; ++r) {
@@ -1582,6 +1595,7 @@ static ear_status_t phase3_16(const Shard &sh, uint16_t *S16, const CUtensorMap 
     total += mode == MODE_LIST ? all : mode == MODE_LIST_CROSS ? cross : all - cross;
   }
   if (total == 0) return EAR_OK;
+  if (reserve < 0) reserve = lookahead_reserve(total, sh.nt - 1);
   TileJob16 J{S16, sh.Np, 0, k, sh.nt, mode, 0, 0, sh.d_rows, sh.d_pre, sh.nown, mk, posk};
   J.posk1 = posk1;
   int s3 = prof_begin(PK_FW_P3_16, st);
@@ -1610,7 +1624,6 @@ static ear_status_t fw_sharded16(std::vector<Shard *> &sh, int32_t Np, ear_comm_
   cudaEvent_t ev_cross, ev_pivot;
   EAR_TRY(side_stream(&side, &ev_cross, &ev_pivot));
   const bool lookahead = env_int("EAR_FW16_LOOKAHEAD", 1) != 0;
-  const int reserve = env_int("EAR_FW16_RESERVE", 4);
   const size_t R = sh.size();
   std::vector<uint16_t *> S16(R, nullptr);
   int32_t *prow = nullptr, *flag = nullptr;
@@ -1698,7 +1711,7 @@ static ear_status_t fw_sharded16(std::vector<Shard *> &sh, int32_t Np, ear_comm_
     e = cudaEventRecord(ev_pivot, side);   // recorded even after an error: the main stream waits for it
     if (s == EAR_OK && e != cudaSuccess) { set_error("fw_sharded16: %s", cudaGetErrorString(e)); s = EAR_ECUDA; }
     for (size_t r = 0; r < R && s == EAR_OK; ++r)
-      s = phase3_16(*sh[r], S16[r], A, B, k, MODE_LIST_REST, st, reserve);
+      s = phase3_16(*sh[r], S16[r], A, B, k, MODE_LIST_REST, st, -1);
     e = cudaStreamWaitEvent(st, ev_pivot, 0);
     if (s == EAR_OK && e != cudaSuccess) { set_error("fw_sharded16: %s", cudaGetErrorString(e)); s = EAR_ECUDA; }
   }
