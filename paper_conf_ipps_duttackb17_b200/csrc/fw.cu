@@ -1220,14 +1220,14 @@ int grid_for(int64_t n) { return (int)std::max<int64_t>(1, std::min<int64_t>(cei
 // CTA slots the rest-of-round launch leaves to the next round's pivot chain.  The persistent,
 // dynamically scheduled tile kernel frees no slot before it drains, so the chain's phase-2 tiles (one
 // pivot row, p2 tiles) run on the reserved slots alongside the rest (rest tiles): enough slots that
-// they finish no later, p2 / R <= rest / (slots - R), plus one for phase 1.  EAR_FW16_RESERVE
-// overrides (measured on cfg4's single-GPU FW: 4 best, profiles/r01y_fw16_dyn.jsonl -- this rule
-// gives 5-6 there and ~28 at 8 ranks, where a rank's rest is 8x smaller).
+// they finish no later, p2 / R <= rest / (slots - R).  EAR_FW16_RESERVE overrides (measured on cfg4's
+// single-GPU FW: 4 best, profiles/r01y_fw16_dyn.jsonl -- the rule gives 4 there, 5 on the re-reduced
+// BCC root piece and ~27 for a rank of 8, whose rest is 8x smaller; profiles/r01z_rank_timing_cfg4.jsonl).
 int lookahead_reserve(int64_t rest, int64_t p2) {
   const int forced = env_int("EAR_FW16_RESERVE", -1);
   if (forced >= 0) return forced;
   const int64_t slots = (int64_t)std::max(g_num_sms, 1) * 3;
-  const int64_t r = (slots * p2 + rest + p2 - 1) / std::max<int64_t>(rest + p2, 1) + 1;
+  const int64_t r = (slots * p2 + rest + p2 - 1) / std::max<int64_t>(rest + p2, 1);
   return (int)std::min<int64_t>(std::max<int64_t>(r, 1), slots / 2);
 }
 
