@@ -1127,6 +1127,8 @@ using Fw16TileS = Fw16Cfg<32, 2, 3, 16, 128, 1, 1, 1>;
 using Fw16TileS3 = Fw16Cfg<32, 3, 3, 16, 128, 1, 1, 1>;
 using Fw16TileD = Fw16Cfg<32, 2, 3, 16, 128, 1, 1, 0, 1>;
 using Fw16TileD0 = Fw16Cfg<32, 2, 3, 16, 128, 0, 1, 0, 1>;
+using Fw16TileD3 = Fw16Cfg<32, 3, 3, 16, 128, 0, 1, 0, 1>;
+using Fw16TileD16 = Fw16Cfg<16, 4, 3, 16, 128, 0, 1, 0, 1>;
 
 // development knobs (tools/): EAR_FW16_LOOKAHEAD=0 disables the lookahead, EAR_FW16_RESERVE sets the
 // CTA slots the rest-of-round launch leaves free for the next round's pivot work (default 4: with the
@@ -1193,7 +1195,10 @@ ear_status_t launch16_cfg(const CUtensorMap &mA, const CUtensorMap &mB, TileJob1
   return EAR_OK;
 }
 
-int fw16_kc() { return env_int("EAR_FW16_VARIANT", 0) == 2 ? Fw16TileL4::kKC : Fw16Tile::kKC; }
+int fw16_kc() {
+  const int v = env_int("EAR_FW16_VARIANT", 0);
+  return v == 2 ? Fw16TileL4::kKC : v == 11 ? Fw16TileD16::kKC : Fw16Tile::kKC;
+}
 
 // EAR_FW16_VARIANT (development knob, tools/lab_fw16_*.sh): 0 = Fw16Tile; static tile assignment:
 // 1 = last-arriver refill, 2 = 4-stage ring of 16-deep chunks, 3 = 3-stage ring, 4 = refill + C prefetch
@@ -1212,6 +1217,8 @@ ear_status_t launch16(const CUtensorMap &mA, const CUtensorMap &mB, TileJob16 J,
   if (variant == 7) return launch16_cfg<Fw16TileS3>(mA, mB, J, nblocks, st, reserve);
   if (variant == 8) return launch16_cfg<Fw16TileD>(mA, mB, J, nblocks, st, reserve);
   if (variant == 9) return launch16_cfg<Fw16TileD0>(mA, mB, J, nblocks, st, reserve);
+  if (variant == 10) return launch16_cfg<Fw16TileD3>(mA, mB, J, nblocks, st, reserve);
+  if (variant == 11) return launch16_cfg<Fw16TileD16>(mA, mB, J, nblocks, st, reserve);
   return launch16_cfg<CF>(mA, mB, J, nblocks, st, reserve);
 }
 
