@@ -118,8 +118,10 @@ __global__ void __launch_bounds__(NT, 1) k_fw_phase1(int32_t *T, int64_t ldt) {
 // MODE_CROSS / MODE_REST (single-GPU lookahead, round k): the upper tiles of row/column k+1 (without
 // column k), and all upper tiles outside rows/columns k and k+1; together they are MODE_UPPER.
 // MODE_LIST_CROSS / MODE_LIST_REST: the same split of a rank's MODE_LIST tiles (sharded lookahead).
+// MODE_PIECES: phase 2 on the pivot-row pieces a rank contributes (owner-side phase 2, sharded FW):
+// tiles (k, orow[i]) for the mk owned rows above k, then (k, k+1 ..) when the rank owns row k (posk).
 enum { MODE_PIVOT_ROW = 0, MODE_UPPER = 1, MODE_LIST = 2, MODE_CROSS = 3, MODE_REST = 4, MODE_LIST_CROSS = 5,
-       MODE_LIST_REST = 6 };
+       MODE_LIST_REST = 6, MODE_PIECES = 7 };
 
 // Tile-kernel configuration: k-chunk depth, TMA ring depth, CTAs per SM, kk-loop unroll.
 template <int KC_, int ST_, int MINB_, int UNR_>
@@ -231,6 +233,12 @@ __device__ __forceinline__ void decode_tile(const TileJob &J, int64_t idx, int &
     ti = (int)a < k ? (int)a : (int)a + skip;
     tj = (int)b < k ? (int)b : (int)b + skip;
     lr = ti - J.ti0;
+    return;
+  }
+  if (J.mode == MODE_PIECES) {   // C: the rank's pieces of the pivot row block (lr 0)
+    ti = k;
+    tj = (int)idx < J.mk ? J.orow[idx] : k + 1 + ((int)idx - J.mk);
+    lr = 0;
     return;
   }
   if (J.mode == MODE_LIST_CROSS) {   // row k+1's tiles (if owned), then tile (ti, k+1) of owned rows ti < k
@@ -364,6 +372,19 @@ __global__ void __launch_bounds__(NT, CF::MINB) k_fw_tiles(const __grid_constant
 
 __global__ void k_fill(int32_t *p, int64_t n, int32_t v) {
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) p[i] = v;
+}
+
+__global__ void k_fill16(uint16_t *p, int64_t n2, uint32_t v2) {   // n2 u16 pairs
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n2; i += (int64_t)gridDim.x * blockDim.x)
+    reinterpret_cast<uint32_t *>(p)[i] = v2;
+}
+
+// u16 block -> int32 (the values are capped 16-bit distances, C16 included), n % 4 == 0
+__global__ void k_widen16(const uint16_t *__restrict__ P16, int32_t *__restrict__ P32, int64_t n) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n / 4; i += (int64_t)gridDim.x * blockDim.x) {
+    const uint2 v = reinterpret_cast<const uint2 *>(P16)[i];
+    reinterpret_cast<int4 *>(P32)[i] = make_int4(v.x & 0xFFFF, v.x >> 16, v.y & 0xFFFF, v.y >> 16);
+  }
 }
 
 // Pivot-row block <-> a rank's owned storage, round k (prow: 128 x Np, leading dimension Np).
@@ -1602,7 +1623,7 @@ static ear_status_t phase3_16(const Shard &sh, uint16_t *S16, const CUtensorMap 
     total += mode == MODE_LIST ? all : mode == MODE_LIST_CROSS ? cross : all - cross;
   }
   if (total == 0) return EAR_OK;
-  if (reserve < 0) reserve = lookahead_reserve(total, sh.nt - 1);
+  if (reserve < 0) reserve = lookahead_reserve(total, (sh.nt - 1 + sh.P - 1) / sh.P);   // owner-side phase 2
   TileJob16 J{S16, sh.Np, 0, k, sh.nt, mode, 0, 0, sh.d_rows, sh.d_pre, sh.nown, mk, posk};
   J.posk1 = posk1;
   int s3 = prof_begin(PK_FW_P3_16, st);
@@ -1636,7 +1657,13 @@ static ear_status_t fw_sharded16(std::vector<Shard *> &sh, int32_t Np, ear_comm_
   int32_t *prow = nullptr, *flag = nullptr;
   uint16_t *p16 = nullptr;   // two 128 x Np buffers (round parity), as Pd
   uint32_t *Pd = nullptr;
+  uint16_t *L16 = nullptr, *ptile = nullptr;   // this rank's pivot-row pieces; the broadcast pivot tile
+  uint32_t *Ld = nullptr;                      // L16 duplicated (phase-2 B operand)
+  const int P = comm ? comm->nranks : (int)sh.size();
   bool ok = cudaMallocAsync((void **)&prow, sizeof(int32_t) * (size_t)TILE * Np, st) == cudaSuccess &&
+            cudaMallocAsync((void **)&L16, sizeof(uint16_t) * (size_t)TILE * Np, st) == cudaSuccess &&
+            cudaMallocAsync((void **)&Ld, sizeof(uint32_t) * (size_t)TILE * Np, st) == cudaSuccess &&
+            cudaMallocAsync((void **)&ptile, sizeof(uint16_t) * TILE * TILE, st) == cudaSuccess &&
             cudaMallocAsync((void **)&p16, 2 * sizeof(uint16_t) * (size_t)TILE * Np, st) == cudaSuccess &&
             cudaMallocAsync((void **)&Pd, 2 * sizeof(uint32_t) * (size_t)TILE * Np, st) == cudaSuccess &&
             cudaMallocAsync((void **)&flag, sizeof(int32_t), st) == cudaSuccess;
@@ -1649,6 +1676,9 @@ static ear_status_t fw_sharded16(std::vector<Shard *> &sh, int32_t Np, ear_comm_
     if (prow) cudaFreeAsync(prow, st);
     if (p16) cudaFreeAsync(p16, st);
     if (Pd) cudaFreeAsync(Pd, st);
+    if (L16) cudaFreeAsync(L16, st);
+    if (Ld) cudaFreeAsync(Ld, st);
+    if (ptile) cudaFreeAsync(ptile, st);
     if (flag) cudaFreeAsync(flag, st);
   };
   if (!ok) {   // no room for the 16-bit copies: the int32 schedule runs
@@ -1658,8 +1688,9 @@ static ear_status_t fw_sharded16(std::vector<Shard *> &sh, int32_t Np, ear_comm_
   }
   const int KC = fw16_kc();
   const int64_t nblk = (int64_t)TILE * Np;
-  CUtensorMap mA[2], mB[2];
-  ear_status_t s = EAR_OK;
+  CUtensorMap mA[2], mB[2], mL, mLd;
+  ear_status_t s = make_map_t(&mL, CU_TENSOR_MAP_DATA_TYPE_UINT16, 2, L16, TILE, Np, Np, KC);
+  if (s == EAR_OK) s = make_map_t(&mLd, CU_TENSOR_MAP_DATA_TYPE_UINT32, 4, Ld, TILE, Np, Np, KC);
   for (int b = 0; b < 2 && s == EAR_OK; ++b) {
     s = make_map_t(&mA[b], CU_TENSOR_MAP_DATA_TYPE_UINT16, 2, p16 + b * nblk, TILE, Np, Np, KC);
     if (s == EAR_OK) s = make_map_t(&mB[b], CU_TENSOR_MAP_DATA_TYPE_UINT32, 4, Pd + b * nblk, TILE, Np, Np, KC);
@@ -1672,31 +1703,54 @@ static ear_status_t fw_sharded16(std::vector<Shard *> &sh, int32_t Np, ear_comm_
             sh[r]->S, sh[r]->ldd, S16[r], Np, (int64_t)sh[r]->nown * TILE, Np);
     prof_end(sc, st, 0);
   }
-  // round k's pivot chain on stream q: pieces -> exchange -> narrowed block (buffer k & 1) -> phases
-  // 1-2 packed, as fw_single16's pivot() -> scattered back to the owners
+  // round k's pivot chain on stream q, with the phase 2 done by the owners of the pieces:
+  //   every rank copies its pieces of the pivot row block into L (u16, C16 elsewhere -- above every
+  //   capped value, so the MIN exchange ignores it); the owner of row k closes the pivot tile in L
+  //   (phase 1) and broadcasts it (32 KB); every rank applies phase 2 to ITS pieces only (MODE_PIECES,
+  //   B = L duplicated before phase 2, as fw_single16's single-product phase 2); the pieces are
+  //   widened and all-reduced (MIN) into the full phase-2-complete block, which is narrowed into the
+  //   A operand of phase 3 (buffer k & 1), duplicated into its B operand and scattered back to the
+  //   owners.  No phase 2 is computed twice: each tile of the pivot row is updated by its contributor.
   auto chain = [&](int k, cudaStream_t q) -> ear_status_t {
     const bool on_side = q != st;
     uint16_t *P16 = p16 + (k & 1) * nblk;
     uint32_t *Pk = Pd + (k & 1) * nblk;
-    EAR_TRY(fill(prow, nblk, INF, q));
+    EAR_LAUNCH(k_fill16, grid_for(nblk / 2), 256, 0, q)(L16, nblk / 2, (uint32_t)C16 * 0x10001u);
     for (size_t r = 0; r < R; ++r)
-      if (sh[r]->nown > 0) EAR_TRY((shard_xfer_t<uint16_t, int32_t>(*sh[r], S16[r], Np, k, prow, 0, q)));
+      if (sh[r]->nown > 0) EAR_TRY((shard_xfer_t<uint16_t, uint16_t>(*sh[r], S16[r], Np, k, L16, 0, q)));
+    const int o = k % (2 * P), owner = o < P ? o : 2 * P - 1 - o;
+    const bool mine = comm ? comm->rank == owner : true;   // emulated: some shard owns it
+    int s1 = prof_begin(on_side ? PK_FW_SIDE_P1 : PK_FW_P1, q);
+    if (mine) EAR_LAUNCH(k_fw_phase1_16, 1, NT, 0, q)(L16 + (int64_t)k * TILE, Np);
+    prof_end(s1, q, mine ? (double)TILE * TILE * TILE : 0.0);
+    if (comm && P > 1) {   // the closed pivot tile from its owner
+      int sc = prof_begin(PK_COMM, q);
+      const size_t pitch = sizeof(uint16_t) * Np, w = sizeof(uint16_t) * TILE;
+      if (mine) EAR_CUDA_TRY(cudaMemcpy2DAsync(ptile, w, L16 + (int64_t)k * TILE, pitch, w, TILE, cudaMemcpyDeviceToDevice, q));
+      EAR_TRY(comm_bcast(comm, reinterpret_cast<int32_t *>(ptile), TILE * TILE / 2, owner, q));
+      if (!mine) EAR_CUDA_TRY(cudaMemcpy2DAsync(L16 + (int64_t)k * TILE, pitch, ptile, w, w, TILE, cudaMemcpyDeviceToDevice, q));
+      prof_end(sc, q, 0);
+    }
+    int s2 = prof_begin(on_side ? PK_FW_SIDE_P2 : PK_FW_P2, q);
+    EAR_LAUNCH(k_dup16, grid_for(nblk / 4), 256, 0, q)(L16, Np, Ld);
+    double p2 = 0;
+    for (size_t r = 0; r < R; ++r) {
+      int posk, mk;
+      shard_pieces(*sh[r], k, &posk, &mk);
+      const int64_t n2 = mk + (posk >= 0 ? nt - 1 - k : 0);
+      if (n2 == 0) continue;
+      TileJob16 J2{L16, Np, 0, k, nt, MODE_PIECES, 0, 0, sh[r]->d_rows, sh[r]->d_pre, sh[r]->nown, mk, posk};
+      EAR_TRY(launch16<Fw16Tile>(mL, mLd, J2, n2, q));
+      p2 += (double)n2 * TILE * TILE * TILE;
+    }
+    prof_end(s2, q, p2);
+    EAR_LAUNCH(k_widen16, grid_for(nblk / 4), 256, 0, q)(L16, prow, nblk);
     if (comm) {
       int sc = prof_begin(PK_COMM, q);
       EAR_TRY(comm_allreduce_min(comm, prow, nblk, q));
       prof_end(sc, q, 0);
     }
-    EAR_LAUNCH(k_prow_to16, grid_for(nblk / 4), 256, 0, q)(prow, P16, nullptr, nblk);
-    int s1 = prof_begin(on_side ? PK_FW_SIDE_P1 : PK_FW_P1, q);
-    EAR_LAUNCH(k_fw_phase1_16, 1, NT, 0, q)(P16 + (int64_t)k * TILE, Np);
-    prof_end(s1, q, (double)TILE * TILE * TILE);
-    int s2 = prof_begin(on_side ? PK_FW_SIDE_P2 : PK_FW_P2, q);
-    EAR_LAUNCH(k_dup16, grid_for(nblk / 4), 256, 0, q)(P16, Np, Pk);
-    TileJob16 J2{P16, Np, 0, k, nt, MODE_PIVOT_ROW, 0, 0};
-    J2.ti0 = k;
-    EAR_TRY(launch16<Fw16Tile>(mA[k & 1], mB[k & 1], J2, nt - 1, q));
-    EAR_LAUNCH(k_dup16, grid_for(nblk / 4), 256, 0, q)(P16, Np, Pk);
-    prof_end(s2, q, (double)(nt - 1) * TILE * TILE * TILE);
+    EAR_LAUNCH(k_prow_to16, grid_for(nblk / 4), 256, 0, q)(prow, P16, Pk, nblk);
     for (size_t r = 0; r < R; ++r)
       if (sh[r]->nown > 0) EAR_TRY((shard_xfer_t<uint16_t, uint16_t>(*sh[r], S16[r], Np, k, P16, 1, q)));
     return EAR_OK;

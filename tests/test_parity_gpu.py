@@ -68,11 +68,15 @@ def test_cfg2_full(pkg):
     assert_exact(run_full(pkg, g), oracle.apsp(g.n, g.src, g.dst, g.w), "cfg2")
 
 
-def test_cfg4_sampled_rows_full_size(pkg):
+@pytest.mark.parametrize("phase2", ["bcc", "fw"])
+def test_cfg4_sampled_rows_full_size(pkg, phase2):
     """cfg4 at full size (100k vertices, ~30k reduced, 40 GB output) in the bench's launch
-    configuration: apsp_full over all rows, then sampled rows compared with the oracle."""
+    configuration (bench.py's default Phase II is FLAG_BCC: blocks, re-reduced root piece, packed FW
+    with dynamic tiles and lookahead; persistent expansion over all rows), then sampled rows compared
+    with the oracle; also the plain FW on all of G^r."""
     g = gg.config("cfg4")
-    out = pkg.apsp_full(g.n, dev(g.src), dev(g.dst), dev(g.w))
+    flags = pkg.FLAG_BCC if phase2 == "bcc" else 0
+    out = pkg.apsp_full(g.n, dev(g.src), dev(g.dst), dev(g.w), flags=flags)
     torch.cuda.synchronize()
     rng = np.random.default_rng(4)
     rows = np.unique(np.concatenate([[0, 1, g.n - 1], rng.choice(g.n, 45, replace=False)]))
@@ -83,6 +87,7 @@ def test_cfg4_sampled_rows_full_size(pkg):
     cols = torch.as_tensor(rows).cuda().long()
     blk = out[cols][:, cols]
     assert torch.equal(blk, blk.T)
+    assert int(out.diagonal().abs().max().item()) == 0
     del out
     torch.cuda.empty_cache()
 
