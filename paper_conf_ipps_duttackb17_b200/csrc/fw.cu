@@ -578,56 +578,77 @@ __global__ void k_check16_list(const uint16_t *__restrict__ S16, int64_t ld16, c
   if (__syncthreads_or(found) && threadIdx.x == 0) atomicMin(flag, -1);
 }
 
-// closure of the 16-bit pivot tile (ld Np), computed in int32 registers (values <= C16, so sums fit)
+// Closure of the 16-bit pivot tile (ld ldt) in place, packed like the tile kernel: thread (ty, tx)
+// owns rows {ty*4 .. +3, 64 + ty*4 .. +3} as 4 row PAIRS and columns {tx*4 .. +3, 64 + tx*4 .. +3},
+// c[p][q] = (T[i][j], T[i+1][j]); step kk reads row kk from shared memory -- it is also column kk, the
+// tile being symmetric -- as the row-pair operand and, duplicated, as the column operand, so one
+// VIADDMNMX.U16x2 relaxes two entries (values <= C16: sums <= 0xFFFE never wrap, results stay
+// <= C16).  About 60 registers: it fits beside two CTAs of the tile kernel, which the lookahead
+// needs (the int32-register closure took 108 x 256 registers, more than an SM has left then, so it
+// waited for every rest-of-round launch to drain).
 __global__ void __launch_bounds__(NT, 1) k_fw_phase1_16(uint16_t *T, int64_t ldt) {
-  __shared__ __align__(16) int32_t rowbuf[2][TILE];
+  __shared__ __align__(16) uint16_t rowbuf[2][TILE];
   const int tx = threadIdx.x & 15, ty = threadIdx.x >> 4;
-  int32_t c[8][8];
+  uint32_t c[4][8];
 #pragma unroll
-  for (int r = 0; r < 8; ++r) {
-    const int i = (r < 4 ? 0 : 64) + ty * 4 + (r & 3);
-    const uint2 lo = *reinterpret_cast<const uint2 *>(T + (int64_t)i * ldt + tx * 4);
-    const uint2 hi = *reinterpret_cast<const uint2 *>(T + (int64_t)i * ldt + 64 + tx * 4);
-    c[r][0] = lo.x & 0xFFFF; c[r][1] = lo.x >> 16; c[r][2] = lo.y & 0xFFFF; c[r][3] = lo.y >> 16;
-    c[r][4] = hi.x & 0xFFFF; c[r][5] = hi.x >> 16; c[r][6] = hi.y & 0xFFFF; c[r][7] = hi.y >> 16;
+  for (int p = 0; p < 4; ++p) {
+    const int i = (p < 2 ? 0 : 64) + ty * 4 + (p & 1) * 2;
+#pragma unroll
+    for (int h = 0; h < 2; ++h) {
+      const uint2 v = *reinterpret_cast<const uint2 *>(T + (int64_t)i * ldt + h * 64 + tx * 4);
+      const uint2 w = *reinterpret_cast<const uint2 *>(T + (int64_t)(i + 1) * ldt + h * 64 + tx * 4);
+      c[p][h * 4 + 0] = __byte_perm(v.x, w.x, 0x5410);
+      c[p][h * 4 + 1] = __byte_perm(v.x, w.x, 0x7632);
+      c[p][h * 4 + 2] = __byte_perm(v.y, w.y, 0x5410);
+      c[p][h * 4 + 3] = __byte_perm(v.y, w.y, 0x7632);
+    }
   }
-  if (ty == 0) {
-    *reinterpret_cast<int4 *>(&rowbuf[0][tx * 4]) = make_int4(c[0][0], c[0][1], c[0][2], c[0][3]);
-    *reinterpret_cast<int4 *>(&rowbuf[0][64 + tx * 4]) = make_int4(c[0][4], c[0][5], c[0][6], c[0][7]);
-  }
+  if (threadIdx.x < TILE / 4)   // row 0
+    reinterpret_cast<uint2 *>(rowbuf[0])[threadIdx.x] = reinterpret_cast<const uint2 *>(T)[threadIdx.x];
   __syncthreads();
   for (int kk = 0; kk < TILE; ++kk) {
-    const int32_t *rb = rowbuf[kk & 1];
-    const int4 alo = *reinterpret_cast<const int4 *>(rb + ty * 4);
-    const int4 ahi = *reinterpret_cast<const int4 *>(rb + 64 + ty * 4);
-    const int4 blo = *reinterpret_cast<const int4 *>(rb + tx * 4);
-    const int4 bhi = *reinterpret_cast<const int4 *>(rb + 64 + tx * 4);
-    const int32_t a[8] = {alo.x, alo.y, alo.z, alo.w, ahi.x, ahi.y, ahi.z, ahi.w};
-    const int32_t b[8] = {blo.x, blo.y, blo.z, blo.w, bhi.x, bhi.y, bhi.z, bhi.w};
+    const uint16_t *rb = rowbuf[kk & 1];
+    const uint2 alo = *reinterpret_cast<const uint2 *>(rb + ty * 4);        // rows ty*4 .. +3 (pairs)
+    const uint2 ahi = *reinterpret_cast<const uint2 *>(rb + 64 + ty * 4);
+    const uint2 blo = *reinterpret_cast<const uint2 *>(rb + tx * 4);        // columns tx*4 .. +3
+    const uint2 bhi = *reinterpret_cast<const uint2 *>(rb + 64 + tx * 4);
+    const uint32_t a[4] = {alo.x, alo.y, ahi.x, ahi.y};
+    const uint32_t b[8] = {__byte_perm(blo.x, 0, 0x1010), __byte_perm(blo.x, 0, 0x3232),
+                           __byte_perm(blo.y, 0, 0x1010), __byte_perm(blo.y, 0, 0x3232),
+                           __byte_perm(bhi.x, 0, 0x1010), __byte_perm(bhi.x, 0, 0x3232),
+                           __byte_perm(bhi.y, 0, 0x1010), __byte_perm(bhi.y, 0, 0x3232)};
 #pragma unroll
-    for (int r = 0; r < 8; ++r)
+    for (int p = 0; p < 4; ++p)
 #pragma unroll
-      for (int q = 0; q < 8; ++q) c[r][q] = mp(a[r], b[q], c[r][q]);
-    const int nk = kk + 1;
+      for (int q = 0; q < 8; ++q) c[p][q] = __viaddmin_u16x2(a[p], b[q], c[p][q]);
+    const int nk = kk + 1;   // its owner publishes row nk for the next step
     if (nk < TILE && ty == ((nk & 63) >> 2)) {
-      const int rr = (nk & 3) + (nk >= 64 ? 4 : 0);
-      int32_t *wb = rowbuf[nk & 1];
+      const int p = ((nk & 3) >> 1) + (nk >= 64 ? 2 : 0), hi = nk & 1;
+      uint16_t *wb = rowbuf[nk & 1];
 #pragma unroll
-      for (int r = 0; r < 8; ++r) {
-        if (r == rr) {
-          *reinterpret_cast<int4 *>(wb + tx * 4) = make_int4(c[r][0], c[r][1], c[r][2], c[r][3]);
-          *reinterpret_cast<int4 *>(wb + 64 + tx * 4) = make_int4(c[r][4], c[r][5], c[r][6], c[r][7]);
+      for (int pp = 0; pp < 4; ++pp) {
+        if (pp == p) {
+          const uint32_t sel = hi ? 0x7632 : 0x5410;
+          *reinterpret_cast<uint2 *>(wb + tx * 4) =
+              make_uint2(__byte_perm(c[pp][0], c[pp][1], sel), __byte_perm(c[pp][2], c[pp][3], sel));
+          *reinterpret_cast<uint2 *>(wb + 64 + tx * 4) =
+              make_uint2(__byte_perm(c[pp][4], c[pp][5], sel), __byte_perm(c[pp][6], c[pp][7], sel));
         }
       }
     }
     __syncthreads();
   }
 #pragma unroll
-  for (int r = 0; r < 8; ++r) {
-    const int i = (r < 4 ? 0 : 64) + ty * 4 + (r & 3);
-    auto pk = [&](int q) { return (uint32_t)min(c[r][q], (int32_t)C16) | ((uint32_t)min(c[r][q + 1], (int32_t)C16) << 16); };
-    *reinterpret_cast<uint2 *>(T + (int64_t)i * ldt + tx * 4) = make_uint2(pk(0), pk(2));
-    *reinterpret_cast<uint2 *>(T + (int64_t)i * ldt + 64 + tx * 4) = make_uint2(pk(4), pk(6));
+  for (int p = 0; p < 4; ++p) {
+    const int i = (p < 2 ? 0 : 64) + ty * 4 + (p & 1) * 2;
+#pragma unroll
+    for (int h = 0; h < 2; ++h) {
+      const uint32_t *cc = &c[p][h * 4];
+      *reinterpret_cast<uint2 *>(T + (int64_t)i * ldt + h * 64 + tx * 4) =
+          make_uint2(__byte_perm(cc[0], cc[1], 0x5410), __byte_perm(cc[2], cc[3], 0x5410));
+      *reinterpret_cast<uint2 *>(T + (int64_t)(i + 1) * ldt + h * 64 + tx * 4) =
+          make_uint2(__byte_perm(cc[0], cc[1], 0x7632), __byte_perm(cc[2], cc[3], 0x7632));
+    }
   }
 }
 
@@ -1150,6 +1171,8 @@ using Fw16TileD = Fw16Cfg<32, 2, 3, 16, 128, 1, 1, 0, 1>;
 using Fw16TileD0 = Fw16Cfg<32, 2, 3, 16, 128, 0, 1, 0, 1>;
 using Fw16TileD3 = Fw16Cfg<32, 3, 3, 16, 128, 0, 1, 0, 1>;
 using Fw16TileD16 = Fw16Cfg<16, 4, 3, 16, 128, 0, 1, 0, 1>;
+using Fw16TileD2x4 = Fw16Cfg<32, 4, 2, 16, 128, 0, 1, 0, 1>;
+using Fw16TileD2x3 = Fw16Cfg<32, 3, 2, 16, 128, 0, 1, 0, 1>;
 
 // development knobs (tools/): EAR_FW16_LOOKAHEAD=0 disables the lookahead, EAR_FW16_RESERVE sets the
 // CTA slots the rest-of-round launch leaves free for the next round's pivot work (default 4: with the
@@ -1240,6 +1263,8 @@ ear_status_t launch16(const CUtensorMap &mA, const CUtensorMap &mB, TileJob16 J,
   if (variant == 9) return launch16_cfg<Fw16TileD0>(mA, mB, J, nblocks, st, reserve);
   if (variant == 10) return launch16_cfg<Fw16TileD3>(mA, mB, J, nblocks, st, reserve);
   if (variant == 11) return launch16_cfg<Fw16TileD16>(mA, mB, J, nblocks, st, reserve);
+  if (variant == 12) return launch16_cfg<Fw16TileD2x4>(mA, mB, J, nblocks, st, reserve);
+  if (variant == 13) return launch16_cfg<Fw16TileD2x3>(mA, mB, J, nblocks, st, reserve);
   return launch16_cfg<CF>(mA, mB, J, nblocks, st, reserve);
 }
 
