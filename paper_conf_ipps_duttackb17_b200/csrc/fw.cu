@@ -203,6 +203,15 @@ __device__ __forceinline__ void tma_load_2d(void *dst, const CUtensorMap *map, i
       : "memory");
 }
 
+__device__ __forceinline__ void tma_load_2d_hint(void *dst, const CUtensorMap *map, int32_t c0, int32_t c1, uint64_t *bar,
+                                                 uint64_t policy) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1, {%2, %3}], [%4], %5;\n" ::"r"(
+          smem_u32(dst)),
+      "l"(reinterpret_cast<uint64_t>(map)), "r"(c0), "r"(c1), "r"(smem_u32(bar)), "l"(policy)
+      : "memory");
+}
+
 // decode the tile index into (ti, tj) and the local tile row lr of C
 __device__ __forceinline__ void decode_tile(const TileJob &J, int64_t idx, int &ti, int &tj, int &lr) {
   const int k = J.k;
@@ -679,14 +688,14 @@ struct TileJob16 {
 // of thread 0 waiting on an 'empty' barrier at the start of each chunk (which ties warp 0 to the
 // slowest warp every chunk).
 template <int KC, int STAGES, int MINB, int UNR, int NTH = 256, int PFC = 0, int LAR = 0, int SPIN = 0,
-          int DYN = 0>
+          int DYN = 0, int HINT = 0>
 struct Fw16Cfg {
   static constexpr int NCHUNK = TILE / KC;
   static constexpr int A_CHUNK = KC * TILE;   // u16 elements
   static constexpr int B_CHUNK = KC * TILE;   // u32 elements
   static constexpr int SMEM = STAGES * (A_CHUNK * 2 + B_CHUNK * 4) + 2 * STAGES * 8 + STAGES * 4 + 8;
   static constexpr int kKC = KC, kSTAGES = STAGES, kMINB = MINB, kUNR = UNR, kNTH = NTH, kPFC = PFC, kLAR = LAR;
-  static constexpr int kSPIN = SPIN, kDYN = DYN;
+  static constexpr int kSPIN = SPIN, kDYN = DYN, kHINT = HINT;
   static constexpr int RPH = 256 * 2 / NTH;   // row pairs per 64-row half owned by a thread (2 or 4)
 };
 
@@ -930,8 +939,15 @@ __global__ void __launch_bounds__(CF::kNTH, CF::kMINB)
     int pti, ptj, plr;
     decode16(J, t, pti, ptj, plr);
     mbar_arrive_tx(&full[st], CF::A_CHUNK * 2 + CF::B_CHUNK * 4);
-    tma_load_2d(sA + st * CF::A_CHUNK, &tmA, pti * TILE, J.a_row0 + kc * KC, &full[st]);
-    tma_load_2d(sB + st * CF::B_CHUNK, &tmB, ptj * TILE, kc * KC, &full[st]);
+    if (CF::kHINT) {   // the pivot row block stays in L2 while the C tiles stream through it
+      uint64_t pol;
+      asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
+      tma_load_2d_hint(sA + st * CF::A_CHUNK, &tmA, pti * TILE, J.a_row0 + kc * KC, &full[st], pol);
+      tma_load_2d_hint(sB + st * CF::B_CHUNK, &tmB, ptj * TILE, kc * KC, &full[st], pol);
+    } else {
+      tma_load_2d(sA + st * CF::A_CHUNK, &tmA, pti * TILE, J.a_row0 + kc * KC, &full[st]);
+      tma_load_2d(sB + st * CF::B_CHUNK, &tmB, ptj * TILE, kc * KC, &full[st]);
+    }
   };
   if (tid == 0) {
     for (int s = 0; s < STAGES; ++s) {
@@ -961,8 +977,10 @@ __global__ void __launch_bounds__(CF::kNTH, CF::kMINB)
       const int i = row_of(r2);
 #pragma unroll
       for (int h = 0; h < 2; ++h) {
-        const uint2 a = *reinterpret_cast<const uint2 *>(Ct + (int64_t)i * J.ldc + h * 64 + tx * 4);
-        const uint2 b = *reinterpret_cast<const uint2 *>(Ct + (int64_t)(i + 1) * J.ldc + h * 64 + tx * 4);
+        const uint2 *pa = reinterpret_cast<const uint2 *>(Ct + (int64_t)i * J.ldc + h * 64 + tx * 4);
+        const uint2 *pb = reinterpret_cast<const uint2 *>(Ct + (int64_t)(i + 1) * J.ldc + h * 64 + tx * 4);
+        const uint2 a = CF::kHINT ? __ldcs(pa) : *pa;
+        const uint2 b = CF::kHINT ? __ldcs(pb) : *pb;
         c[r2][h * 4 + 0] = __byte_perm(a.x, b.x, 0x5410);
         c[r2][h * 4 + 1] = __byte_perm(a.x, b.x, 0x7632);
         c[r2][h * 4 + 2] = __byte_perm(a.y, b.y, 0x5410);
@@ -1023,10 +1041,11 @@ __global__ void __launch_bounds__(CF::kNTH, CF::kMINB)
 #pragma unroll
       for (int h = 0; h < 2; ++h) {
         const uint32_t *cc = &c[r2][h * 4];
-        *reinterpret_cast<uint2 *>(Ct + (int64_t)i * J.ldc + h * 64 + tx * 4) =
-            make_uint2(__byte_perm(cc[0], cc[1], 0x5410), __byte_perm(cc[2], cc[3], 0x5410));
-        *reinterpret_cast<uint2 *>(Ct + (int64_t)(i + 1) * J.ldc + h * 64 + tx * 4) =
-            make_uint2(__byte_perm(cc[0], cc[1], 0x7632), __byte_perm(cc[2], cc[3], 0x7632));
+        uint2 *qa = reinterpret_cast<uint2 *>(Ct + (int64_t)i * J.ldc + h * 64 + tx * 4);
+        uint2 *qb = reinterpret_cast<uint2 *>(Ct + (int64_t)(i + 1) * J.ldc + h * 64 + tx * 4);
+        const uint2 va = make_uint2(__byte_perm(cc[0], cc[1], 0x5410), __byte_perm(cc[2], cc[3], 0x5410));
+        const uint2 vb = make_uint2(__byte_perm(cc[0], cc[1], 0x7632), __byte_perm(cc[2], cc[3], 0x7632));
+        if (CF::kHINT) { __stcs(qa, va); __stcs(qb, vb); } else { *qa = va; *qb = vb; }
       }
     }
     if (J.mirror && ti != tj) {
@@ -1173,6 +1192,7 @@ using Fw16TileD3 = Fw16Cfg<32, 3, 3, 16, 128, 0, 1, 0, 1>;
 using Fw16TileD16 = Fw16Cfg<16, 4, 3, 16, 128, 0, 1, 0, 1>;
 using Fw16TileD2x4 = Fw16Cfg<32, 4, 2, 16, 128, 0, 1, 0, 1>;
 using Fw16TileD2x3 = Fw16Cfg<32, 3, 2, 16, 128, 0, 1, 0, 1>;
+using Fw16TileDH = Fw16Cfg<32, 2, 3, 16, 128, 0, 1, 0, 1, 1>;
 
 // development knobs (tools/): EAR_FW16_LOOKAHEAD=0 disables the lookahead, EAR_FW16_RESERVE sets the
 // CTA slots the rest-of-round launch leaves free for the next round's pivot work (default 4: with the
@@ -1265,6 +1285,7 @@ ear_status_t launch16(const CUtensorMap &mA, const CUtensorMap &mB, TileJob16 J,
   if (variant == 11) return launch16_cfg<Fw16TileD16>(mA, mB, J, nblocks, st, reserve);
   if (variant == 12) return launch16_cfg<Fw16TileD2x4>(mA, mB, J, nblocks, st, reserve);
   if (variant == 13) return launch16_cfg<Fw16TileD2x3>(mA, mB, J, nblocks, st, reserve);
+  if (variant == 14) return launch16_cfg<Fw16TileDH>(mA, mB, J, nblocks, st, reserve);
   return launch16_cfg<CF>(mA, mB, J, nblocks, st, reserve);
 }
 
