@@ -1,6 +1,7 @@
 """Small end-to-end runs for compute-sanitizer (memcheck / racecheck / synccheck): every kernel of the
-library on graphs small enough for the instrumented run -- FW (single + emulated sharding), SSSP,
-expansion (aligned and scalar store paths), query mode, Phase I with pure cycles."""
+library on graphs small enough for the instrumented run -- packed and int32 FW (single + emulated
+sharding with the owner-side phase 2 and lookahead), blocks with a re-reduced piece, SSSP, expansion
+(aligned and scalar store paths), query mode, Phase I with pure cycles."""
 import sys
 
 import numpy as np
@@ -11,11 +12,16 @@ import paper_conf_ipps_duttackb17_b200 as ea  # noqa: E402
 from paper_conf_ipps_duttackb17_b200 import graphgen as gg  # noqa: E402
 
 dev = lambda a: torch.as_tensor(np.ascontiguousarray(a, dtype=np.int32)).cuda()  # noqa: E731
-for g in [gg.corner_cases(5, n_target=300), gg.torus(12, 12, 150, seed=1), gg.cycle(40, seed=2)]:
-    for flags in (0, ea.FLAG_SSSP):
+from tests.test_bcc_gpu import decorated_grid  # noqa: E402  (a big block that is reduced again)
+
+for g in [gg.corner_cases(5, n_target=300), gg.torus(12, 12, 150, seed=1), gg.cycle(40, seed=2),
+          decorated_grid(18, 0.35, 1)]:
+    for flags in (0, ea.FLAG_SSSP, ea.FLAG_BCC, ea.FLAG_FW32):
         out = ea.apsp_full(g.n, dev(g.src), dev(g.dst), dev(g.w), flags=flags)
     plan = ea.ear_decompose(g.n, dev(g.src), dev(g.dst), dev(g.w))
     D = ea.apsp_reduced_emulated(plan, 2)
+    D3 = ea.apsp_reduced_emulated(plan, 3)   # packed sharded FW: owner-side phase 2, lookahead
+    ea.apsp_reduced_rank_timing(plan, 2, 1)
     big = torch.zeros((g.n, g.n + 3), dtype=torch.int32, device="cuda")
     ea.expand_ears(plan, D, 0, g.n, out=big[:, 1:1 + g.n])
     s = dev(np.arange(g.n)); t = dev(np.arange(g.n)[::-1].copy())
