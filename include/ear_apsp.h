@@ -267,6 +267,9 @@ typedef struct {
                                   there -- they OVERLAP phase 3 of round k, so this is not additive */
   double rereduce_ms;          /* EAR_FLAG_BCC: Phase I + Phase III of re-reduced big pieces */
   double bcc_prepare_ms;       /* EAR_FLAG_BCC: block structure of G^r (first solve of a plan only) */
+  int64_t fw16_prechecked;     /* packed FWs abandoned after round 3: the eccentricity of reduced vertex 0
+                                  (one SSSP row, overlapped with rounds 0-3) already reached the 16-bit cap;
+                                  each is also counted in fw16_fallbacks */
 } ear_profile_t;
 
 void ear_profile_enable(int32_t on);

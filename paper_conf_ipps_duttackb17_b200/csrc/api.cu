@@ -171,7 +171,7 @@ ear_status_t apsp_reduced(ear_plan_t p, int32_t *d_D, int64_t ldd, ear_comm_t co
     const bool allow16 = !(p->flags & EAR_FLAG_FW32);
     const int32_t *lab = nullptr;
     if (allow16) EAR_TRY(reduced_labels(p, Np, st, &lab));
-    return fw_single(d_D, ldd, Np, st, lab, p->n_reduced, allow16);
+    return fw_single(d_D, ldd, Np, st, lab, p->n_reduced, allow16, p);
   }
   // with a communicator -- even one of a single rank -- d_D holds this rank's owned tile rows
   // (zig-zag assignment, ascending) and the sharded schedule with its NCCL calls runs

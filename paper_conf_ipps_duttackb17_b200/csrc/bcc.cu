@@ -732,7 +732,7 @@ static ear_status_t reduce_solve(const ear_plan_s *p, int32_t n, int64_t m, cons
   if (s == EAR_OK && !inner) {
     if (!comm) {
       s = fw_init_D(q, D, Np, Np, 0, Np, st);
-      if (s == EAR_OK) s = fw_single(D, Np, Np, st, nullptr, q->n_reduced, allow16);   // connected
+      if (s == EAR_OK) s = fw_single(D, Np, Np, st, nullptr, q->n_reduced, allow16, q);   // connected
     } else {
       const std::vector<int32_t> own = shard_rows(Np / TILE, P, comm->rank);
       int32_t *S = nullptr;

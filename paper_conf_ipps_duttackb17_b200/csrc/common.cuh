@@ -93,6 +93,7 @@ void prof_fw16(bool used);   // one 16-bit FW attempt: used, or fell back to int
 void count_launch(int n = 1);
 int prof_begin(int kind, cudaStream_t s);                // -1 when profiling is off
 void prof_end(int slot, cudaStream_t s, double work);
+void prof_fw16_precheck();   // a packed FW abandoned after round 0 by its cap precheck
 // launch one of the library's kernels and count it: EAR_LAUNCH(k, grid, block, smem, stream)(args);
 #define EAR_LAUNCH(k, g, b, sm, st) ::ear::count_launch(), k<<<(g), (b), (sm), (st)>>>
 // decompose.cu
@@ -103,7 +104,7 @@ void plan_free(ear_plan_s *plan);
 ear_status_t fw_init_D(const ear_plan_s *plan, int32_t *D, int64_t ldd, int32_t Np, int32_t row0,
                        int32_t rows, cudaStream_t stream);
 ear_status_t fw_single(int32_t *D, int64_t ldd, int32_t Np, cudaStream_t stream, const int32_t *lab = nullptr,
-                       int32_t n_real = 0, bool allow16 = false);
+                       int32_t n_real = 0, bool allow16 = false, ear_plan_s *plan = nullptr);
 ear_status_t reduced_labels(ear_plan_s *p, int32_t Np, cudaStream_t st, const int32_t **out);
 // row-block sharding: rank r owns the tile rows ti with (ti mod 2P) in {r, 2P-1-r} (zig-zag), stored
 // ascending as 128-row blocks

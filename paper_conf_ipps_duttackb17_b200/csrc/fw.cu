@@ -499,6 +499,17 @@ __global__ void k_check16(const uint16_t *__restrict__ D16, int32_t Np, const in
   if (__syncthreads_or(found) && threadIdx.x == 0) atomicOr(bad, 1);
 }
 
+// largest finite entry of a distance row (the cap precheck of fw_single16)
+__global__ void k_row_far(const int32_t *__restrict__ row, int32_t n, int32_t *far) {
+  int32_t m = 0;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    const int32_t v = row[i];
+    if (v < INF) m = max(m, v);
+  }
+  m = __reduce_max_sync(0xFFFFFFFFu, m);
+  if ((threadIdx.x & 31) == 0) atomicMax(far, m);
+}
+
 __global__ void k_from16(const uint16_t *__restrict__ D16, int32_t Np, int32_t *__restrict__ D, int64_t ldd) {
   const int64_t total = (int64_t)Np * (Np / 4);
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
@@ -1336,7 +1347,7 @@ ear_status_t side_stream(cudaStream_t *side, cudaEvent_t *ev_cross, cudaEvent_t 
 // phase 3 waits for both.  The two streams touch disjoint tiles (the rest skips rows/columns k, k+1)
 // and alternate between two Pd buffers, so the serial phases 1-2 leave the critical path.
 ear_status_t fw_single16(int32_t *D, int64_t ldd, int32_t Np, const int32_t *lab, int32_t n_real, bool *done,
-                         cudaStream_t st) {
+                         cudaStream_t st, ear_plan_s *plan) {
   *done = false;
   if (!g_num_sms) {
     int dev = 0;
@@ -1389,7 +1400,42 @@ ear_status_t fw_single16(int32_t *D, int64_t ldd, int32_t Np, const int32_t *lab
     return EAR_OK;
   };
   if (s == EAR_OK && nt > 0) s = pivot(0, st);
+  // Cap precheck, overlapped with rounds 0-3: the exact distance row of reduced vertex 0 by one
+  // single-source SSSP on a helper stream.  Its eccentricity is a lower bound on the largest finite
+  // distance; when it already reaches the cap, a connected pair is capped for sure, so the packed FW
+  // is abandoned after round 3 instead of running to the end and being thrown away (cfg5: diameter
+  // ~42.8k).  Vertex 0 sits at a corner of the spatially coherent labellings, so its eccentricity is
+  // close to the diameter.  Only with a plan (plain FW, re-reduced pieces) and a large FW.
+  bool pre = s == EAR_OK && plan && nt >= 64 && env_int("EAR_FW16_PRECHECK", 1) != 0;
+  cudaStream_t hs = nullptr;
+  cudaEvent_t ev_pre = nullptr;
+  int32_t *pre_row = nullptr, *pre_res = nullptr;
+  static int32_t *h_pre = nullptr;   // pinned
+  if (pre) {
+    pre = cudaStreamCreateWithFlags(&hs, cudaStreamNonBlocking) == cudaSuccess &&
+          cudaEventCreateWithFlags(&ev_pre, cudaEventDisableTiming) == cudaSuccess &&
+          (h_pre || cudaMallocHost((void **)&h_pre, sizeof(int32_t)) == cudaSuccess) &&
+          cudaMallocAsync((void **)&pre_row, sizeof(int32_t) * ((size_t)Np + 1), hs) == cudaSuccess;
+    if (pre) {
+      pre_res = pre_row + Np;
+      cudaMemsetAsync(pre_res, 0, sizeof(int32_t), hs);
+      pre = sssp_rows(plan, pre_row, Np, Np, 0, 1, nullptr, hs) == EAR_OK;
+    }
+    if (pre) {
+      EAR_LAUNCH(k_row_far, grid_for(n_real), 256, 0, hs)(pre_row, n_real, pre_res);
+      pre = cudaMemcpyAsync(h_pre, pre_res, sizeof(int32_t), cudaMemcpyDeviceToHost, hs) == cudaSuccess &&
+            cudaEventRecord(ev_pre, hs) == cudaSuccess;
+    }
+    if (!pre) cudaGetLastError();
+  }
+  bool hopeless = false;
   for (int k = 0; k < nt && s == EAR_OK; ++k) {
+    if (pre && k == 4) {   // rounds 0-3 (~4 ms at cfg4 sizes) cover the SSSP: the host rarely waits
+      if (cudaEventSynchronize(ev_pre) == cudaSuccess && *h_pre >= (int32_t)C16) {
+        hopeless = true;
+        break;
+      }
+    }
     TileJob16 J{D16, Np, k * TILE, k, nt, MODE_UPPER, 1, 0};
     const int64_t nup = (int64_t)(nt - 1) * nt / 2;
     if (!lookahead || k + 1 == nt) {
@@ -1422,8 +1468,16 @@ ear_status_t fw_single16(int32_t *D, int64_t ldd, int32_t Np, const int32_t *lab
     }
   }
   if (s != EAR_OK) cudaStreamWaitEvent(st, ev_pivot, 0);   // never leave side work behind the frees
+  if (hs) {
+    cudaStreamSynchronize(hs);
+    if (pre_row) cudaFreeAsync(pre_row, hs);
+    cudaStreamSynchronize(hs);
+    cudaStreamDestroy(hs);
+    cudaEventDestroy(ev_pre);
+  }
   int32_t h_bad = 1;
-  if (s == EAR_OK) {
+  if (s == EAR_OK && hopeless) prof_fw16_precheck();
+  if (s == EAR_OK && !hopeless) {
     int sc = prof_begin(PK_FW16_CONV, st);
     cudaMemsetAsync(bad, 0, sizeof(int32_t), st);
     EAR_LAUNCH(k_check16, grid_for((int64_t)Np * (Np / 8)), 256, 0, st)(D16, Np, lab, n_real, bad);
@@ -1467,10 +1521,10 @@ ear_status_t fw_init_D(const ear_plan_s *plan, int32_t *D, int64_t ldd, int32_t 
 // its result is kept when no connected pair (labels lab over [0, n_real), or one component when lab is
 // NULL) reached the 16-bit cap; otherwise, or without allow16, the int32 FW below runs.
 ear_status_t fw_single(int32_t *D, int64_t ldd, int32_t Np, cudaStream_t st, const int32_t *lab, int32_t n_real,
-                       bool allow16) {
+                       bool allow16, ear_plan_s *plan) {
   if (allow16 && Np >= 2 * TILE) {
     bool done = false;
-    EAR_TRY(fw_single16(D, ldd, Np, lab, n_real, &done, st));
+    EAR_TRY(fw_single16(D, ldd, Np, lab, n_real, &done, st, plan));
     prof_fw16(done);
     if (done) return EAR_OK;
   }

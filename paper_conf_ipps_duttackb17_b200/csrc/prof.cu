@@ -36,6 +36,11 @@ cudaEvent_t get_event() {
 
 void count_launch(int n) { g_launches.fetch_add(n, std::memory_order_relaxed); }
 
+void prof_fw16_precheck() {
+  std::lock_guard<std::mutex> lk(g_mu);
+  g_acc.fw16_prechecked++;
+}
+
 void prof_fw16(bool used) {
   std::lock_guard<std::mutex> lk(g_mu);
   if (used) g_acc.fw16_used++; else g_acc.fw16_fallbacks++;

@@ -56,7 +56,8 @@ class _Profile(ctypes.Structure):
                 ("compose_bytes", ctypes.c_double), ("fw16_used", ctypes.c_int64), ("fw16_fallbacks", ctypes.c_int64),
                 ("fw16_conv_ms", ctypes.c_double), ("fw_phase3_16_ms", ctypes.c_double),
                 ("fw_phase3_16_minplus", ctypes.c_double), ("fw_side_ms", ctypes.c_double),
-                ("rereduce_ms", ctypes.c_double), ("bcc_prepare_ms", ctypes.c_double)]
+                ("rereduce_ms", ctypes.c_double), ("bcc_prepare_ms", ctypes.c_double),
+                ("fw16_prechecked", ctypes.c_int64)]
 
 
 class _BccInfo(ctypes.Structure):

@@ -213,3 +213,40 @@ def test_sharded16_without_lookahead(pkg, P, monkeypatch):
     assert prof["fw16_used"] == 1
     assert np.array_equal(d_la, d_serial)
     assert_exact(d_serial, oracle_on_terminals(g), f"sharded16 serial P={P}")
+
+
+def test_cap_precheck_abandons_hopeless_fw16(pkg):
+    """A reduced graph large enough for the cap precheck (>= 64 tiles) whose corner vertex is already
+    farther than the cap from something: the packed FW is abandoned after round 3 and the int32 FW
+    gives the exact result (sampled rows against the oracle)."""
+    g = ladder(4200, 100, seed=11)              # 8,400 vertices in a 2 x 4,200 ladder, distances ~420k
+    plan = pkg.ear_decompose(g.n, dev(g.src), dev(g.dst), dev(g.w))
+    D = pkg.alloc_D(plan)
+    pkg.profile_reset()
+    pkg.profile_enable(True)
+    pkg.apsp_reduced(plan, D)
+    torch.cuda.synchronize()
+    prof = pkg.profile_read()
+    pkg.profile_enable(False)
+    assert plan.info().n_reduced_padded // 128 >= 64
+    assert prof["fw16_prechecked"] == 1 and prof["fw16_fallbacks"] == 1 and prof["fw16_used"] == 0
+    r = oracle.reduce_graph(g.n, g.src, g.dst, g.w)
+    T = np.nonzero(r.term)[0]
+    rows = np.random.default_rng(2).choice(len(T), 12, replace=False)
+    ref = oracle.apsp_rows(g.n, g.src, g.dst, g.w, T[rows])[:, T]
+    assert_exact(D[torch.as_tensor(rows).cuda().long()][:, :len(T)].cpu().numpy(), ref, "precheck fallback")
+
+
+def test_cap_precheck_keeps_short_fw16(pkg):
+    """cfg2 (20k vertices, 7,917 reduced: 62 tiles -> no precheck) and a large short-distance ladder
+    (precheck passes): the packed result is kept."""
+    g = ladder(4200, 3, seed=12)                # distances ~12.6k < cap
+    plan = pkg.ear_decompose(g.n, dev(g.src), dev(g.dst), dev(g.w))
+    D = pkg.alloc_D(plan)
+    pkg.profile_reset()
+    pkg.profile_enable(True)
+    pkg.apsp_reduced(plan, D)
+    torch.cuda.synchronize()
+    prof = pkg.profile_read()
+    pkg.profile_enable(False)
+    assert prof["fw16_prechecked"] == 0 and prof["fw16_used"] == 1

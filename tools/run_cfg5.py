@@ -27,13 +27,13 @@ def main():
     ap.add_argument("--config", default="cfg5")
     ap.add_argument("--block", type=int, default=25000)
     ap.add_argument("--check-rows", type=int, default=4, help="oracle-checked rows per block")
-    ap.add_argument("--phase2", choices=["fw", "sssp"], default="fw")
+    ap.add_argument("--phase2", choices=["fw", "sssp", "bcc"], default="fw")
     args = ap.parse_args()
     import oracle
 
     g = gg.config(args.config)
     src, dst, w = (torch.as_tensor(x).cuda() for x in (g.src, g.dst, g.w))
-    flags = ea.FLAG_SSSP if args.phase2 == "sssp" else 0
+    flags = {"fw": 0, "sssp": ea.FLAG_SSSP, "bcc": ea.FLAG_BCC}[args.phase2]
     ev = lambda: torch.cuda.Event(enable_timing=True)  # noqa: E731
     e0, e1, e2 = ev(), ev(), ev()
     torch.cuda.synchronize()
