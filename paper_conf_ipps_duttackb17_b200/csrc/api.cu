@@ -195,7 +195,7 @@ ear_status_t apsp_reduced(ear_plan_t p, int32_t *d_D, int64_t ldd, ear_comm_t co
     const bool allow16 = !(p->flags & EAR_FLAG_FW32);
     const int32_t *lab = nullptr;
     if (s == EAR_OK && allow16) s = reduced_labels(p, Np, st, &lab);
-    if (s == EAR_OK) s = fw_sharded_auto(d_D, ldd, Np, comm, lab, p->n_reduced, allow16, st);
+    if (s == EAR_OK) s = fw_sharded_auto(d_D, ldd, Np, comm, lab, p->n_reduced, allow16, st, p);
   }
   cudaFreeAsync(d_rows, st);
   return s;

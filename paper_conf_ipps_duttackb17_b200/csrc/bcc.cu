@@ -743,7 +743,7 @@ static ear_status_t reduce_solve(const ear_plan_s *p, int32_t n, int64_t m, cons
       }
       for (size_t j = 0; j < own.size() && s == EAR_OK; ++j)
         s = fw_init_D(q, S + (int64_t)j * TILE * Np, Np, Np, own[j] * TILE, TILE, st);
-      if (s == EAR_OK) s = fw_sharded_auto(S, Np, Np, comm, nullptr, q->n_reduced, allow16, st);
+      if (s == EAR_OK) s = fw_sharded_auto(S, Np, Np, comm, nullptr, q->n_reduced, allow16, st, q);
       if (s == EAR_OK) s = fw_sharded_gather(S, Np, Np, D, Np, comm, st);
       if (S) cudaFreeAsync(S, st);
     }

@@ -111,7 +111,7 @@ ear_status_t reduced_labels(ear_plan_s *p, int32_t Np, cudaStream_t st, const in
 ear_status_t fw_sharded(int32_t *S, int64_t ldd, int32_t Np, ear_comm_s *comm, cudaStream_t stream);
 // the 16-bit sharded schedule first (allow16; lab / n_real as for fw_single), else fw_sharded
 ear_status_t fw_sharded_auto(int32_t *S, int64_t ldd, int32_t Np, ear_comm_s *comm, const int32_t *lab,
-                             int32_t n_real, bool allow16, cudaStream_t stream);
+                             int32_t n_real, bool allow16, cudaStream_t stream, ear_plan_s *plan = nullptr);
 ear_status_t fw_sharded_gather(const int32_t *S, int64_t ldd, int32_t Np, int32_t *Df, int64_t ldf, ear_comm_s *comm,
                                cudaStream_t stream);
 ear_status_t fw_rank_timing(const ear_plan_s *plan, int32_t Np, int32_t P, int32_t rank, cudaStream_t stream);

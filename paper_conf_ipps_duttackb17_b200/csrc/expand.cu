@@ -31,6 +31,7 @@
 // with D resident in L2 the same kernel runs at ~90 % of the copy bandwidth.
 // k_same_chain: the P:107 along-chain patch, one warp per row, touching only same-chain entries.
 #include <algorithm>
+#include <cstdlib>
 
 #include "common.cuh"
 
@@ -72,6 +73,7 @@ __device__ __forceinline__ int32_t *row_ptr(int32_t *base, int32_t r, uint32_t l
 // items instead of a partial wave of whole row groups.
 struct ExpandWork {
   int32_t *counter;
+  int32_t segmajor;   // > 0: every row group in segmajor column segments, items segment-major
   int32_t n_full, n_items, nseg, seg_w;
 };
 
@@ -97,7 +99,12 @@ __global__ void __launch_bounds__(NT, EXP_MINB) k_expand(const int32_t *__restri
   const int32_t item = item_sh;
   if (item >= W.n_items) break;
   int32_t rg = item, col_b = 0, col_e = n;
-  if (item >= W.n_full) {
+  if (W.segmajor > 0) {
+    const int32_t groups = W.n_items / W.segmajor;
+    rg = item % groups;
+    col_b = (item / groups) * W.seg_w;
+    col_e = min(n, col_b + W.seg_w);
+  } else if (item >= W.n_full) {
     rg = W.n_full + (item - W.n_full) / W.nseg;
     col_b = ((item - W.n_full) % W.nseg) * W.seg_w;
     col_e = min(n, col_b + W.seg_w);
@@ -276,6 +283,11 @@ __global__ void k_query_pairs(const int32_t *__restrict__ D, int64_t ldd, const 
 
 bool g_attr_set = false;
 
+int env_int_ex(const char *name, int dflt) {
+  const char *e = getenv(name);
+  return e ? atoi(e) : dflt;
+}
+
 }  // namespace
 
 ear_status_t expand(const ear_plan_s *plan, const int32_t *D, int64_t ldd, int32_t row_begin, int32_t row_end,
@@ -301,6 +313,12 @@ ear_status_t expand(const ear_plan_s *plan, const int32_t *D, int64_t ldd, int32
   const int32_t nsplit = std::min(groups, slots);
   W.n_full = groups - nsplit;
   W.n_items = W.n_full + nsplit * W.nseg;
+  static const int segs = env_int_ex("EAR_EXPAND_SEGS", 0);   // development knob: segment-major items
+  if (segs > 0) {
+    W.seg_w = (int32_t)round_up(ceil_div(plan->n, segs), CHUNK);
+    W.segmajor = (int32_t)ceil_div(plan->n, W.seg_w);
+    W.n_items = groups * W.segmajor;
+  }
   EAR_CUDA_TRY(cudaMallocAsync((void **)&W.counter, sizeof(int32_t), st));
   EAR_CUDA_TRY(cudaMemsetAsync(W.counter, 0, sizeof(int32_t), st));
   const unsigned grid = (unsigned)std::min<int64_t>(W.n_items, slots);

@@ -1337,6 +1337,48 @@ ear_status_t side_stream(cudaStream_t *side, cudaEvent_t *ev_cross, cudaEvent_t 
   return EAR_OK;
 }
 
+// Cap precheck of the packed FW: one single-source SSSP row of reduced vertex 0 on a helper stream,
+// its eccentricity (a lower bound on the largest finite distance) read back asynchronously.  start()
+// does nothing without a plan, for a small FW (< 64 tiles) or with EAR_FW16_PRECHECK=0; hopeless()
+// waits for the row and says whether it reached the cap.  The row is exact and deterministic, so every
+// rank of a sharded FW takes the same decision without a collective.
+struct Precheck {
+  cudaStream_t hs = nullptr;
+  cudaEvent_t ev = nullptr;
+  int32_t *row = nullptr;
+  bool on = false;
+  static int32_t *host() {   // pinned, one per process (one FW at a time)
+    static int32_t *h = nullptr;
+    if (!h && cudaMallocHost((void **)&h, sizeof(int32_t)) != cudaSuccess) h = nullptr;
+    return h;
+  }
+  void start(ear_plan_s *plan, int32_t Np, int32_t n_real, int nt) {
+    if (!plan || nt < 64 || env_int("EAR_FW16_PRECHECK", 1) == 0 || !host()) return;
+    on = cudaStreamCreateWithFlags(&hs, cudaStreamNonBlocking) == cudaSuccess &&
+         cudaEventCreateWithFlags(&ev, cudaEventDisableTiming) == cudaSuccess &&
+         cudaMallocAsync((void **)&row, sizeof(int32_t) * ((size_t)Np + 1), hs) == cudaSuccess &&
+         cudaMemsetAsync(row + Np, 0, sizeof(int32_t), hs) == cudaSuccess &&
+         sssp_rows(plan, row, Np, Np, 0, 1, nullptr, hs) == EAR_OK;
+    if (on) {
+      EAR_LAUNCH(k_row_far, grid_for(n_real), 256, 0, hs)(row, n_real, row + Np);
+      on = cudaMemcpyAsync(host(), row + Np, sizeof(int32_t), cudaMemcpyDeviceToHost, hs) == cudaSuccess &&
+           cudaEventRecord(ev, hs) == cudaSuccess;
+    }
+    if (!on) cudaGetLastError();
+  }
+  bool hopeless() { return on && cudaEventSynchronize(ev) == cudaSuccess && *host() >= (int32_t)C16; }
+  void finish() {
+    if (!hs) return;
+    cudaStreamSynchronize(hs);
+    if (row) cudaFreeAsync(row, hs);
+    cudaStreamSynchronize(hs);
+    cudaStreamDestroy(hs);
+    if (ev) cudaEventDestroy(ev);
+    hs = nullptr;
+  }
+  ~Precheck() { finish(); }
+};
+
 // The packed 16-bit FW on a copy of D (see C16 above).  *done = false (D untouched) when a connected
 // pair reached the cap; the caller then runs the int32 FW.  Synchronises the stream once (the check).
 //
@@ -1406,35 +1448,13 @@ ear_status_t fw_single16(int32_t *D, int64_t ldd, int32_t Np, const int32_t *lab
   // is abandoned after round 3 instead of running to the end and being thrown away (cfg5: diameter
   // ~42.8k).  Vertex 0 sits at a corner of the spatially coherent labellings, so its eccentricity is
   // close to the diameter.  Only with a plan (plain FW, re-reduced pieces) and a large FW.
-  bool pre = s == EAR_OK && plan && nt >= 64 && env_int("EAR_FW16_PRECHECK", 1) != 0;
-  cudaStream_t hs = nullptr;
-  cudaEvent_t ev_pre = nullptr;
-  int32_t *pre_row = nullptr, *pre_res = nullptr;
-  static int32_t *h_pre = nullptr;   // pinned
-  if (pre) {
-    pre = cudaStreamCreateWithFlags(&hs, cudaStreamNonBlocking) == cudaSuccess &&
-          cudaEventCreateWithFlags(&ev_pre, cudaEventDisableTiming) == cudaSuccess &&
-          (h_pre || cudaMallocHost((void **)&h_pre, sizeof(int32_t)) == cudaSuccess) &&
-          cudaMallocAsync((void **)&pre_row, sizeof(int32_t) * ((size_t)Np + 1), hs) == cudaSuccess;
-    if (pre) {
-      pre_res = pre_row + Np;
-      cudaMemsetAsync(pre_res, 0, sizeof(int32_t), hs);
-      pre = sssp_rows(plan, pre_row, Np, Np, 0, 1, nullptr, hs) == EAR_OK;
-    }
-    if (pre) {
-      EAR_LAUNCH(k_row_far, grid_for(n_real), 256, 0, hs)(pre_row, n_real, pre_res);
-      pre = cudaMemcpyAsync(h_pre, pre_res, sizeof(int32_t), cudaMemcpyDeviceToHost, hs) == cudaSuccess &&
-            cudaEventRecord(ev_pre, hs) == cudaSuccess;
-    }
-    if (!pre) cudaGetLastError();
-  }
+  Precheck pc;
+  if (s == EAR_OK) pc.start(plan, Np, n_real, nt);
   bool hopeless = false;
   for (int k = 0; k < nt && s == EAR_OK; ++k) {
-    if (pre && k == 4) {   // rounds 0-3 (~4 ms at cfg4 sizes) cover the SSSP: the host rarely waits
-      if (cudaEventSynchronize(ev_pre) == cudaSuccess && *h_pre >= (int32_t)C16) {
-        hopeless = true;
-        break;
-      }
+    if (k == 4 && pc.hopeless()) {   // rounds 0-3 (~4 ms at cfg4 sizes) cover the SSSP: the host rarely waits
+      hopeless = true;
+      break;
     }
     TileJob16 J{D16, Np, k * TILE, k, nt, MODE_UPPER, 1, 0};
     const int64_t nup = (int64_t)(nt - 1) * nt / 2;
@@ -1468,13 +1488,7 @@ ear_status_t fw_single16(int32_t *D, int64_t ldd, int32_t Np, const int32_t *lab
     }
   }
   if (s != EAR_OK) cudaStreamWaitEvent(st, ev_pivot, 0);   // never leave side work behind the frees
-  if (hs) {
-    cudaStreamSynchronize(hs);
-    if (pre_row) cudaFreeAsync(pre_row, hs);
-    cudaStreamSynchronize(hs);
-    cudaStreamDestroy(hs);
-    cudaEventDestroy(ev_pre);
-  }
+  pc.finish();
   int32_t h_bad = 1;
   if (s == EAR_OK && hopeless) prof_fw16_precheck();
   if (s == EAR_OK && !hopeless) {
@@ -1739,7 +1753,8 @@ static ear_status_t phase3_16(const Shard &sh, uint16_t *S16, const CUtensorMap 
 // tiles, the narrowed block and its duplicate alternate between two buffers by round parity, and round
 // k+1's phase 3 waits for the chain.
 static ear_status_t fw_sharded16(std::vector<Shard *> &sh, int32_t Np, ear_comm_s *comm, const int32_t *lab,
-                                 int32_t n_real, bool *done, cudaStream_t st, bool timing_only = false) {
+                                 int32_t n_real, bool *done, cudaStream_t st, bool timing_only = false,
+                                 ear_plan_s *plan = nullptr) {
   *done = false;
   const int nt = Np / TILE;
   if (nt < 2) return EAR_OK;
@@ -1856,7 +1871,14 @@ static ear_status_t fw_sharded16(std::vector<Shard *> &sh, int32_t Np, ear_comm_
     return EAR_OK;
   };
   if (s == EAR_OK) s = chain(0, st);
+  Precheck pc;   // as fw_single16's; every rank decides the same
+  if (s == EAR_OK && !timing_only) pc.start(plan, Np, n_real, nt);
+  bool hopeless = false;
   for (int k = 0; k < nt && s == EAR_OK; ++k) {
+    if (k == 4 && pc.hopeless()) {
+      hopeless = true;
+      break;
+    }
     const CUtensorMap &A = mA[k & 1], &B = mB[k & 1];
     if (!lookahead || k + 1 == nt) {
       for (size_t r = 0; r < R && s == EAR_OK; ++r) s = phase3_16(*sh[r], S16[r], A, B, k, MODE_LIST, st);
@@ -1875,6 +1897,13 @@ static ear_status_t fw_sharded16(std::vector<Shard *> &sh, int32_t Np, ear_comm_
       s = phase3_16(*sh[r], S16[r], A, B, k, MODE_LIST_REST, st, -1);
     e = cudaStreamWaitEvent(st, ev_pivot, 0);
     if (s == EAR_OK && e != cudaSuccess) { set_error("fw_sharded16: %s", cudaGetErrorString(e)); s = EAR_ECUDA; }
+  }
+  pc.finish();
+  if (s == EAR_OK && hopeless) {   // the int32 schedule runs on the untouched int32 rows
+    prof_fw16_precheck();
+    release();
+    EAR_CUDA_TRY(cudaGetLastError());
+    return EAR_OK;
   }
   int32_t h_flag = -1;
   if (s == EAR_OK && timing_only) {   // apsp_reduced_rank_timing: no check, no result
@@ -1913,13 +1942,13 @@ static ear_status_t fw_sharded16(std::vector<Shard *> &sh, int32_t Np, ear_comm_
 // Sharded FW on a rank's owned int32 rows: the 16-bit schedule first (allow16), the int32 one when it
 // did not apply.  lab / n_real as for fw_single.
 ear_status_t fw_sharded_auto(int32_t *S, int64_t ldd, int32_t Np, ear_comm_s *comm, const int32_t *lab,
-                             int32_t n_real, bool allow16, cudaStream_t st) {
+                             int32_t n_real, bool allow16, cudaStream_t st, ear_plan_s *plan) {
   if (allow16 && Np >= 2 * TILE) {
     Shard sh;
     EAR_TRY(shard_setup(&sh, S, ldd, Np, comm->nranks, comm->rank, st));
     std::vector<Shard *> v{&sh};
     bool done = false;
-    ear_status_t s = fw_sharded16(v, Np, comm, lab, n_real, &done, st);
+    ear_status_t s = fw_sharded16(v, Np, comm, lab, n_real, &done, st, false, plan);
     shard_free(&sh, st);
     EAR_TRY(s);
     prof_fw16(done);
@@ -2011,7 +2040,7 @@ ear_status_t fw_sharded_emulated(ear_plan_s *plan, int32_t *D, int64_t ldd, int3
     status = reduced_labels(plan, Np, st, &lab);
     std::vector<Shard *> v;
     for (int r = 0; r < P; ++r) v.push_back(&sh[r]);
-    if (status == EAR_OK) status = fw_sharded16(v, Np, nullptr, lab, plan->n_reduced, &done16, st);
+    if (status == EAR_OK) status = fw_sharded16(v, Np, nullptr, lab, plan->n_reduced, &done16, st, false, plan);
     if (status == EAR_OK) prof_fw16(done16);
   }
   int32_t *prow = nullptr;

@@ -250,3 +250,16 @@ def test_cap_precheck_keeps_short_fw16(pkg):
     prof = pkg.profile_read()
     pkg.profile_enable(False)
     assert prof["fw16_prechecked"] == 0 and prof["fw16_used"] == 1
+
+
+def test_cap_precheck_sharded(pkg):
+    """The sharded packed schedule takes the same precheck (every rank decides alike): abandoned after
+    round 3 for the long ladder, the int32 schedule's result exact (sampled rows)."""
+    g = ladder(4200, 100, seed=13)
+    d, prof = emulated(pkg, g, 3)
+    assert prof["fw16_prechecked"] == 1 and prof["fw16_used"] == 0
+    r = oracle.reduce_graph(g.n, g.src, g.dst, g.w)
+    T = np.nonzero(r.term)[0]
+    rows = np.random.default_rng(3).choice(len(T), 10, replace=False)
+    ref = oracle.apsp_rows(g.n, g.src, g.dst, g.w, T[rows])[:, T]
+    assert_exact(d[rows], ref, "sharded precheck fallback")
