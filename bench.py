@@ -383,7 +383,7 @@ def run_ours(args, rank, world, local_rank):
         barrier()
         e2e = {"value": float(g.n) * g.n * e2e_steps / e2e_s, "unit": UNIT, "h2d_bytes_per_step": 3 * 4 * g.m,
                "d2h_bytes_per_step": 4 * rows * g.n, "steps": e2e_steps,
-               "api": "apsp_full_host (pinned host edge list in, pinned host rows out)"}
+               "api": "apsp_full_host (pinned host edge list in, read in place; pinned host rows out)"}
         del hout
 
     cpu = None

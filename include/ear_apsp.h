@@ -224,6 +224,23 @@ ear_status_t apsp_full_host(int32_t n, int64_t m, const int32_t *h_src, const in
                             const int32_t *h_w, uint32_t flags, int32_t row_begin, int32_t row_end,
                             int32_t *h_out, int64_t ldo, ear_comm_t comm, void *stream);
 
+/* apsp_full_host split in two, so that consecutive problems pipeline: the call returns once Phases I
+ * and II are enqueued on `stream` (it synchronises `stream` once, inside the decomposition), with the
+ * expansion on a job-owned stream and the device -> host copies of the rows on the device's host-copy
+ * stream (one per device, FIFO: the copies of successive jobs into the same h_out land in order), so
+ * that the next job's Phases I-II on `stream` can overlap this job's 4*rows*n bytes of PCIe traffic.
+ * Measured on cfg4 (tools/e2e_pipeline.py): no overlap yet -- the next job's small device -> host
+ * readbacks (Phase I counts, the 16-bit range check) queue on the copy engine behind this job's row
+ * copies, so each job still waits for the previous job's copies.  h_out
+ * and the input arrays must stay valid, and h_out unread, until ear_job_wait(*job) returns; it waits,
+ * frees the job's scratch and returns the job's status.  Errors of the enqueue phase are returned
+ * directly (no job).  Library-owned job handle. */
+typedef struct ear_job_s *ear_job_t;
+ear_status_t apsp_full_host_async(int32_t n, int64_t m, const int32_t *h_src, const int32_t *h_dst,
+                                  const int32_t *h_w, uint32_t flags, int32_t row_begin, int32_t row_end,
+                                  int32_t *h_out, int64_t ldo, ear_comm_t comm, void *stream, ear_job_t *job);
+ear_status_t ear_job_wait(ear_job_t job);
+
 /* ---------------------------------------------------------------- multi-GPU plumbing
  * Contiguous near-equal split of `rows` rows over nranks: rank gets [*begin, *end). */
 void ear_row_block(int32_t rows, int32_t nranks, int32_t rank, int32_t *begin, int32_t *end);

@@ -316,73 +316,152 @@ ear_status_t apsp_full(int32_t n, int64_t m, const int32_t *d_src, const int32_t
   return s;
 }
 
-ear_status_t apsp_full_host(int32_t n, int64_t m, const int32_t *h_src, const int32_t *h_dst, const int32_t *h_w,
-                            uint32_t flags, int32_t row_begin, int32_t row_end, int32_t *h_out, int64_t ldo,
-                            ear_comm_t comm, void *stream) {
+}  // extern "C"
+
+struct ear_job_s {
+  ear_plan_s *plan = nullptr;
+  int32_t *Dfull = nullptr;
+  int32_t *buf[2] = {nullptr, nullptr};
+  cudaStream_t es = nullptr;                      // expansion stream
+  cudaEvent_t ev_fw = nullptr, ready[2] = {nullptr, nullptr}, freed[2] = {nullptr, nullptr}, done = nullptr;
+  ear_status_t status = EAR_OK;
+};
+
+namespace {
+// the device's host-copy stream: every job's D2H copies, in issue order
+cudaStream_t host_copy_stream() {
+  static cudaStream_t cs[64] = {};
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return nullptr;
+  if (!cs[dev] && cudaStreamCreateWithFlags(&cs[dev], cudaStreamNonBlocking) != cudaSuccess) cs[dev] = nullptr;
+  return cs[dev];
+}
+
+void job_release(ear_job_s *j) {
+  if (j->done) cudaEventSynchronize(j->done);
+  // stream-ordered frees only: a cudaFree would synchronise the whole device, i.e. wait for the NEXT
+  // job's Phase II too and serialise the pipeline
+  cudaStream_t fs = j->es ? j->es : cudaStreamPerThread;
+  if (j->Dfull) cudaFreeAsync(j->Dfull, fs);
+  for (int i = 0; i < 2; ++i)
+    if (j->buf[i]) cudaFreeAsync(j->buf[i], fs);
+  cudaStreamSynchronize(fs);
+  for (int i = 0; i < 2; ++i) {
+    if (j->ready[i]) cudaEventDestroy(j->ready[i]);
+    if (j->freed[i]) cudaEventDestroy(j->freed[i]);
+  }
+  if (j->ev_fw) cudaEventDestroy(j->ev_fw);
+  if (j->done) cudaEventDestroy(j->done);
+  if (j->es) cudaStreamDestroy(j->es);
+  if (j->plan) ear_plan_destroy(j->plan);
+  delete j;
+}
+}  // namespace
+
+extern "C" {
+
+ear_status_t apsp_full_host_async(int32_t n, int64_t m, const int32_t *h_src, const int32_t *h_dst, const int32_t *h_w,
+                                  uint32_t flags, int32_t row_begin, int32_t row_end, int32_t *h_out, int64_t ldo,
+                                  ear_comm_t comm, void *stream, ear_job_t *job) {
   cudaStream_t st = (cudaStream_t)stream;
-  if (row_begin < 0 || row_end < row_begin || row_end > n || ldo < n || (m > 0 && (!h_src || !h_dst || !h_w))) {
-    set_error("apsp_full_host: bad arguments");
+  if (!job || row_begin < 0 || row_end < row_begin || row_end > n || ldo < n ||
+      (m > 0 && (!h_src || !h_dst || !h_w)) || (row_end > row_begin && !h_out)) {
+    set_error("apsp_full_host_async: bad arguments");
     return EAR_EINVAL;
   }
-  // 1. edges host -> device
+  *job = nullptr;
+  cudaStream_t cs = host_copy_stream();
+  if (!cs) { set_error("apsp_full_host_async: no copy stream"); return EAR_ECUDA; }
+  // 1. the edges: pinned host arrays are read in place by Phase I's first kernels (zero-copy over
+  // PCIe); others are copied in.  A copy would queue behind the previous job's device -> host row
+  // copies on the copy engines and keep this job's Phases I-II from overlapping them.
+  auto mapped = [](const int32_t *h) -> const int32_t * {
+    cudaPointerAttributes a{};
+    if (cudaPointerGetAttributes(&a, h) != cudaSuccess) { cudaGetLastError(); return nullptr; }
+    return a.type == cudaMemoryTypeHost && a.devicePointer ? static_cast<const int32_t *>(a.devicePointer) : nullptr;
+  };
+  const int32_t *ms = m > 0 ? mapped(h_src) : nullptr, *md = m > 0 ? mapped(h_dst) : nullptr,
+                *mw = m > 0 ? mapped(h_w) : nullptr;
   int32_t *dE = nullptr;
-  const size_t eb = sizeof(int32_t) * (size_t)std::max<int64_t>(m, 1);
-  EAR_CUDA_TRY(cudaMallocAsync((void **)&dE, 3 * eb, st));
-  if (m > 0) {
+  const int32_t *es = ms, *ed = md, *ew = mw;
+  if (m > 0 && !(ms && md && mw)) {
+    const size_t eb = sizeof(int32_t) * (size_t)m;
+    EAR_CUDA_TRY(cudaMallocAsync((void **)&dE, 3 * eb, st));
     EAR_CUDA_TRY(cudaMemcpyAsync(dE, h_src, eb, cudaMemcpyHostToDevice, st));
     EAR_CUDA_TRY(cudaMemcpyAsync(dE + m, h_dst, eb, cudaMemcpyHostToDevice, st));
     EAR_CUDA_TRY(cudaMemcpyAsync(dE + 2 * m, h_w, eb, cudaMemcpyHostToDevice, st));
+    es = dE; ed = dE + m; ew = dE + 2 * m;
   }
-  ear_plan_t p = nullptr;
-  ear_status_t s = ear_decompose(n, m, dE, dE + m, dE + 2 * m, flags, stream, &p);
-  cudaFreeAsync(dE, st);
-  if (s != EAR_OK) return s;
-  // 2. reduced APSP, D kept
-  int32_t *Dfull = nullptr;
-  s = solve_rows(p, row_begin, row_end, nullptr, ldo, comm, st, &Dfull);
+  ear_job_s *j = new ear_job_s;
+  ear_status_t s = ear_decompose(n, m, es, ed, ew, flags, stream, &j->plan);
+  if (dE) cudaFreeAsync(dE, st);
+  // 2. reduced APSP on `stream`, D kept
+  if (s == EAR_OK) s = solve_rows(j->plan, row_begin, row_end, nullptr, ldo, comm, st, &j->Dfull);
   const int32_t P = comm ? comm->nranks : 1;
-  const int32_t Np = padded(p, P);
-  // 3. expansion in row chunks, double-buffered against the device -> host copies
+  const int32_t Np = s == EAR_OK ? padded(j->plan, P) : 0;
+  // 3. expansion on the job's stream, in row chunks double-buffered against the copies
   const int32_t rows = row_end - row_begin;
+  cudaError_t e = cudaSuccess;
+  if (s == EAR_OK) {
+    e = cudaStreamCreateWithFlags(&j->es, cudaStreamNonBlocking);
+    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&j->ev_fw, cudaEventDisableTiming);
+    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&j->done, cudaEventDisableTiming);
+    if (e == cudaSuccess) e = cudaEventRecord(j->ev_fw, st);
+    if (e == cudaSuccess) e = cudaStreamWaitEvent(j->es, j->ev_fw, 0);
+    if (e != cudaSuccess) { set_error("apsp_full_host_async: %s", cudaGetErrorString(e)); s = EAR_ECUDA; }
+  }
   if (s == EAR_OK && rows > 0) {
     int32_t chunk = (int32_t)std::max<int64_t>(32, std::min<int64_t>(rows, (256ll << 20) / (4ll * n)));
     chunk = (int32_t)round_up(chunk, 32);
-    int32_t *buf[2] = {nullptr, nullptr};
-    cudaStream_t cs = nullptr;
-    cudaEvent_t ready[2] = {nullptr, nullptr}, freed[2] = {nullptr, nullptr};
-    cudaError_t e = cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking);
     for (int i = 0; i < 2 && e == cudaSuccess; ++i) {
-      e = cudaMallocAsync((void **)&buf[i], sizeof(int32_t) * (size_t)chunk * n, st);
-      if (e == cudaSuccess) e = cudaEventCreateWithFlags(&ready[i], cudaEventDisableTiming);
-      if (e == cudaSuccess) e = cudaEventCreateWithFlags(&freed[i], cudaEventDisableTiming);
+      e = cudaMallocAsync((void **)&j->buf[i], sizeof(int32_t) * (size_t)chunk * n, j->es);
+      if (e == cudaSuccess) e = cudaEventCreateWithFlags(&j->ready[i], cudaEventDisableTiming);
+      if (e == cudaSuccess) e = cudaEventCreateWithFlags(&j->freed[i], cudaEventDisableTiming);
     }
-    if (e != cudaSuccess) { set_error("apsp_full_host: %s", cudaGetErrorString(e)); s = EAR_ECUDA; }
+    if (e != cudaSuccess) { set_error("apsp_full_host_async: %s", cudaGetErrorString(e)); s = EAR_ECUDA; }
     int it = 0;
     for (int32_t r = row_begin; s == EAR_OK && r < row_end; r += chunk, ++it) {
       const int b = it & 1;
       const int32_t r1 = std::min(row_end, r + chunk);
-      if (it >= 2) cudaStreamWaitEvent(st, freed[b], 0);
-      s = expand(p, Dfull, Np, r, r1, buf[b], n, st);
+      if (it >= 2) cudaStreamWaitEvent(j->es, j->freed[b], 0);
+      s = expand(j->plan, j->Dfull, Np, r, r1, j->buf[b], n, j->es);
       if (s != EAR_OK) break;
-      cudaEventRecord(ready[b], st);
-      cudaStreamWaitEvent(cs, ready[b], 0);
-      e = cudaMemcpy2DAsync(h_out + (int64_t)(r - row_begin) * ldo, sizeof(int32_t) * ldo, buf[b],
+      cudaEventRecord(j->ready[b], j->es);
+      cudaStreamWaitEvent(cs, j->ready[b], 0);
+      e = cudaMemcpy2DAsync(h_out + (int64_t)(r - row_begin) * ldo, sizeof(int32_t) * ldo, j->buf[b],
                             sizeof(int32_t) * n, sizeof(int32_t) * n, r1 - r, cudaMemcpyDeviceToHost, cs);
       if (e != cudaSuccess) { set_error("apsp_full_host D2H: %s", cudaGetErrorString(e)); s = EAR_ECUDA; break; }
-      cudaEventRecord(freed[b], cs);
+      cudaEventRecord(j->freed[b], cs);
     }
-    cudaStreamSynchronize(cs);
-    cudaStreamSynchronize(st);
-    for (int i = 0; i < 2; ++i) {
-      if (buf[i]) cudaFreeAsync(buf[i], st);
-      if (ready[i]) cudaEventDestroy(ready[i]);
-      if (freed[i]) cudaEventDestroy(freed[i]);
-    }
-    if (cs) cudaStreamDestroy(cs);
   }
-  if (Dfull) cudaFreeAsync(Dfull, st);
-  cudaError_t e = cudaStreamSynchronize(st);
-  ear_plan_destroy(p);
+  if (j->done) cudaEventRecord(j->done, cs);
+  if (s != EAR_OK) {
+    cudaStreamSynchronize(st);
+    job_release(j);
+    return s;
+  }
+  *job = j;
+  return EAR_OK;
+}
+
+ear_status_t ear_job_wait(ear_job_t j) {
+  if (!j) { set_error("ear_job_wait: NULL job"); return EAR_EINVAL; }
+  cudaError_t e = cudaSuccess;
+  if (j->done) e = cudaEventSynchronize(j->done);
+  if (e == cudaSuccess && j->es) e = cudaStreamSynchronize(j->es);
+  ear_status_t s = j->status;
+  if (s == EAR_OK && e != cudaSuccess) { set_error("ear_job_wait: %s", cudaGetErrorString(e)); s = EAR_ECUDA; }
+  job_release(j);
+  return s;
+}
+
+ear_status_t apsp_full_host(int32_t n, int64_t m, const int32_t *h_src, const int32_t *h_dst, const int32_t *h_w,
+                            uint32_t flags, int32_t row_begin, int32_t row_end, int32_t *h_out, int64_t ldo,
+                            ear_comm_t comm, void *stream) {
+  ear_job_t j = nullptr;
+  EAR_TRY(apsp_full_host_async(n, m, h_src, h_dst, h_w, flags, row_begin, row_end, h_out, ldo, comm, stream, &j));
+  ear_status_t s = ear_job_wait(j);
+  cudaError_t e = cudaStreamSynchronize((cudaStream_t)stream);
   if (s == EAR_OK && e != cudaSuccess) { set_error("apsp_full_host: %s", cudaGetErrorString(e)); s = EAR_ECUDA; }
   return s;
 }

@@ -85,6 +85,8 @@ SIGNATURES = {
     "ear_query_pairs": (_I32, [_P, _P, _I64, _I64, _P, _P, _P, _P]),
     "apsp_full": (_I32, [_I32, _I64, _P, _P, _P, _U32, _I32, _I32, _P, _I64, _P, _P]),
     "apsp_full_host": (_I32, [_I32, _I64, _P, _P, _P, _U32, _I32, _I32, _P, _I64, _P, _P]),
+    "apsp_full_host_async": (_I32, [_I32, _I64, _P, _P, _P, _U32, _I32, _I32, _P, _I64, _P, _P, ctypes.POINTER(_P)]),
+    "ear_job_wait": (_I32, [_P]),
     "ear_row_block": (None, [_I32, _I32, _I32, ctypes.POINTER(_I32), ctypes.POINTER(_I32)]),
     "ear_comm_unique_id": (_I32, [ctypes.c_char_p]),
     "ear_comm_init": (_I32, [ctypes.c_char_p, _I32, _I32, ctypes.POINTER(_P)]),
@@ -345,6 +347,42 @@ def apsp_full_host(n: int, src: np.ndarray | torch.Tensor, dst, w, out: torch.Te
                                 flags, row_begin, row_end, out.data_ptr(), out.stride(0), _comm_handle(comm),
                                 _stream(stream)), "apsp_full_host")
     return out
+
+
+class HostJob:
+    """An apsp_full_host_async call in flight: wait() returns the filled host tensor."""
+
+    def __init__(self, handle, out, keep):
+        self.handle, self.out, self._keep = handle, out, keep
+
+    def wait(self) -> torch.Tensor:
+        if self.handle is not None:
+            h, self.handle = self.handle, None
+            _check(lib().ear_job_wait(h), "ear_job_wait")
+        return self.out
+
+
+def apsp_full_host_async(n: int, src, dst, w, out: torch.Tensor | None = None, row_begin: int = 0,
+                         row_end: int | None = None, flags: int = 0, comm: Comm | None = None,
+                         stream=None) -> HostJob:
+    """apsp_full_host that returns once Phases I-II are enqueued (the expansion and the row copies
+    complete in the background; the next call's Phases I-II overlap them).  Call .wait() before reading
+    `out`; the host arrays must stay alive until then."""
+    row_end = n if row_end is None else row_end
+    tens = [torch.as_tensor(np.ascontiguousarray(x, dtype=np.int32)) if not isinstance(x, torch.Tensor) else x
+            for x in (src, dst, w)]
+    for t in tens:
+        if t.is_cuda or t.dtype != torch.int32 or not t.is_contiguous():
+            raise EarError("apsp_full_host_async takes contiguous int32 host arrays")
+    if out is None:
+        out = torch.empty((row_end - row_begin, n), dtype=torch.int32, pin_memory=True)
+    if out.is_cuda or out.dtype != torch.int32 or out.stride(1) != 1:
+        raise EarError("out must be a host int32 tensor with unit column stride")
+    h = ctypes.c_void_p()
+    _check(lib().apsp_full_host_async(n, tens[0].numel(), tens[0].data_ptr(), tens[1].data_ptr(), tens[2].data_ptr(),
+                                      flags, row_begin, row_end, out.data_ptr(), out.stride(0), _comm_handle(comm),
+                                      _stream(stream), ctypes.byref(h)), "apsp_full_host_async")
+    return HostJob(h, out, tens)
 
 
 def profile_enable(on: bool = True):

@@ -194,6 +194,24 @@ def test_host_entry_point(pkg):
     assert_exact(out2.numpy(), oracle.apsp_rows(g.n, g.src, g.dst, g.w, np.arange(100, 1333)), "host rows")
 
 
+@pytest.mark.parametrize("flags", [0, "bcc"])
+def test_host_async_pipelined(pkg, flags):
+    """apsp_full_host_async: two problems in flight at once (the second's Phases I-II overlap the
+    first's row copies), into separate host buffers and, in order, into one shared buffer."""
+    fl = pkg.FLAG_BCC if flags == "bcc" else 0
+    g1, g2 = gg.config("cfg1"), gg.corner_cases(77, n_target=900)
+    r1, r2 = oracle.apsp(g1.n, g1.src, g1.dst, g1.w), oracle.apsp(g2.n, g2.src, g2.dst, g2.w)
+    j1 = pkg.apsp_full_host_async(g1.n, g1.src, g1.dst, g1.w, flags=fl)
+    j2 = pkg.apsp_full_host_async(g2.n, g2.src, g2.dst, g2.w, flags=fl)
+    assert_exact(j2.wait().numpy(), r2, "async second")
+    assert_exact(j1.wait().numpy(), r1, "async first")
+    shared = torch.empty((g1.n, g1.n), dtype=torch.int32, pin_memory=True)
+    jobs = [pkg.apsp_full_host_async(g1.n, g1.src, g1.dst, g1.w, out=shared, flags=fl) for _ in range(3)]
+    for j in jobs:
+        j.wait()
+    assert_exact(shared.numpy(), r1, "async shared buffer")
+
+
 # ------------------------------------------------------------------------------ degenerate inputs
 def graph(n, edges):
     from paper_conf_ipps_duttackb17_b200.graphgen import Graph

@@ -28,6 +28,7 @@ def main():
     ap.add_argument("--block", type=int, default=25000)
     ap.add_argument("--check-rows", type=int, default=4, help="oracle-checked rows per block")
     ap.add_argument("--phase2", choices=["fw", "sssp", "bcc"], default="fw")
+    ap.add_argument("--warmup", type=int, default=1, help="untimed Phase II runs before the timed one")
     args = ap.parse_args()
     import oracle
 
@@ -36,6 +37,13 @@ def main():
     flags = {"fw": 0, "sssp": ea.FLAG_SSSP, "bcc": ea.FLAG_BCC}[args.phase2]
     ev = lambda: torch.cuda.Event(enable_timing=True)  # noqa: E731
     e0, e1, e2 = ev(), ev(), ev()
+    if args.warmup:   # one untimed Phase II: first-use costs (the stream-ordered pool's growth to tens of GB)
+        wp = ea.ear_decompose(g.n, src, dst, w, flags=flags)
+        Dw = ea.alloc_D(wp)
+        ea.apsp_reduced(wp, Dw)
+        torch.cuda.synchronize()
+        del Dw
+        wp.destroy()
     torch.cuda.synchronize()
     t_start = time.perf_counter()
     e0.record()
@@ -67,7 +75,7 @@ def main():
     wall = time.perf_counter() - t_start
     total_ms = ms_dec + ms_p2 + ms_exp
     print(json.dumps({"config": args.config, "n": g.n, "m": g.m, "n_reduced": info.n_reduced,
-                      "phase2": args.phase2, "decompose_ms": ms_dec, "phase2_ms": ms_p2, "expand_ms": ms_exp,
+                      "phase2": args.phase2, "warmup": args.warmup, "decompose_ms": ms_dec, "phase2_ms": ms_p2, "expand_ms": ms_exp,
                       "device_ms": total_ms, "entries_per_s_device": g.n * g.n / (total_ms / 1e3),
                       "output_bytes": 4 * g.n * g.n, "D_bytes": 4 * info.n_reduced_padded ** 2,
                       "expand_GBps": 4.0 * g.n * g.n / (ms_exp / 1e3) / 1e9,
