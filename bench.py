@@ -15,8 +15,10 @@ and the output (40 GB) are far larger than L2, so no flush is needed between ste
 
 Rank 0 prints one JSON line.  Extra keys: roofline (dominant kernel = FW phase-3 min-plus tile
 kernel, ALU bound), roofline_expand (HBM bound), cpu_baseline (the CPU oracle on a bounded sample,
-rank 0 at N = 1 only), e2e (the same metric through the host-buffer C-ABI call apsp_full_host with
-every step's H2D edge upload and D2H copy of the output rows), clocks, gpu_launches, phases_ms.
+rank 0 at N = 1 only), e2e (the same metric through the host-buffer C-ABI calls with every step's
+H2D edge upload and D2H copy of the output rows: by default K jobs of apsp_full_host_async pipelined one
+deep -- job i+1's Phases I-II overlap job i's expansion and row copies -- into two pinned output buffers;
+--e2e-mode sync times the synchronous apsp_full_host), clocks, gpu_launches, phases_ms.
 
 --impl reference runs the CPU oracle (Dijkstra from every source of a bounded sample of sources on
 all host cores) as the reference arm; under torchrun only rank 0 runs it.
@@ -31,6 +33,8 @@ import subprocess
 import sys
 import threading
 import time
+
+import psutil
 
 ROOT = os.path.dirname(os.path.abspath(__file__))
 if ROOT not in sys.path:
@@ -369,22 +373,37 @@ def run_ours(args, rank, world, local_rank):
         hs = torch.as_tensor(g.src).pin_memory()
         hd = torch.as_tensor(g.dst).pin_memory()
         hw = torch.as_tensor(g.w).pin_memory()
-        hout = torch.empty((rows, g.n), dtype=torch.int32, pin_memory=True)
         e2e_steps = max(1, min(args.steps, args.e2e_steps))
-        ea.apsp_full_host(g.n, hs, hd, hw, out=hout, row_begin=r0, row_end=r1, flags=flags, comm=comm,
+        out_bytes = 4 * rows * g.n
+        pipelined = args.e2e_mode == "pipelined"
+        # two pinned output buffers when the host has room (job i+1 never lands in job i's rows)
+        nbuf = 2 if pipelined and psutil.virtual_memory().available > 2.5 * out_bytes else 1
+        houts = [torch.empty((rows, g.n), dtype=torch.int32, pin_memory=True) for _ in range(nbuf)]
+        ea.apsp_full_host(g.n, hs, hd, hw, out=houts[0], row_begin=r0, row_end=r1, flags=flags, comm=comm,
                           stream=stream)
         barrier()
         t = time.perf_counter()
-        for _ in range(e2e_steps):
-            ea.apsp_full_host(g.n, hs, hd, hw, out=hout, row_begin=r0, row_end=r1, flags=flags, comm=comm,
-                              stream=stream)
+        if pipelined:   # one job in flight ahead: job i+1's Phases I-II overlap job i's expansion + row copies
+            prev = None
+            for i in range(e2e_steps):
+                job = ea.apsp_full_host_async(g.n, hs, hd, hw, out=houts[i % nbuf], row_begin=r0, row_end=r1,
+                                              flags=flags, comm=comm, stream=stream)
+                if prev is not None:
+                    prev.wait()
+                prev = job
+            prev.wait()
+        else:
+            for _ in range(e2e_steps):
+                ea.apsp_full_host(g.n, hs, hd, hw, out=houts[0], row_begin=r0, row_end=r1, flags=flags, comm=comm,
+                                  stream=stream)
         torch.cuda.synchronize()
         e2e_s = max_over_ranks(time.perf_counter() - t, world, dev)
         barrier()
         e2e = {"value": float(g.n) * g.n * e2e_steps / e2e_s, "unit": UNIT, "h2d_bytes_per_step": 3 * 4 * g.m,
-               "d2h_bytes_per_step": 4 * rows * g.n, "steps": e2e_steps,
-               "api": "apsp_full_host (pinned host edge list in, read in place; pinned host rows out)"}
-        del hout
+               "d2h_bytes_per_step": out_bytes, "steps": e2e_steps, "mode": args.e2e_mode, "host_out_buffers": nbuf,
+               "api": ("apsp_full_host_async + ear_job_wait, one job in flight ahead" if pipelined else "apsp_full_host")
+               + " (pinned host edge list in, read in place; pinned host rows out)"}
+        del houts
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
@@ -432,7 +451,9 @@ def main():
                          "blocked FW on all of G^r, or per-source SSSP (SURVEY 8.f NEXT 2)")
     ap.add_argument("--fw32", action="store_true", help="int32 FW throughout (EAR_FLAG_FW32)")
     ap.add_argument("--no-e2e", action="store_true")
-    ap.add_argument("--e2e-steps", type=int, default=2)
+    ap.add_argument("--e2e-steps", type=int, default=4)
+    ap.add_argument("--e2e-mode", choices=["sync", "pipelined"], default="pipelined",
+                    help="e2e calls: synchronous apsp_full_host, or async jobs pipelined one deep")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-alt", action="store_true", help="skip the one-off SSSP Phase II timing")
     ap.add_argument("--cpu-seconds", type=float, default=15.0)

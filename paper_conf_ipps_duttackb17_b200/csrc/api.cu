@@ -186,8 +186,9 @@ ear_status_t apsp_reduced(ear_plan_t p, int32_t *d_D, int64_t ldd, ear_comm_t co
   } else {
     std::vector<int32_t> rows(nown);
     if (nown > 0) {
-      cudaError_t e = cudaMemcpyAsync(rows.data(), d_rows, sizeof(int32_t) * nown, cudaMemcpyDeviceToHost, st);
-      if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+      Readback rb(st);
+      cudaError_t e = rb.get(rows.data(), d_rows, sizeof(int32_t) * nown);
+      if (e == cudaSuccess) e = rb.sync();
       if (e != cudaSuccess) { set_error("apsp_reduced: %s", cudaGetErrorString(e)); s = EAR_ECUDA; }
     }
     for (int32_t b = 0; b < nown && s == EAR_OK; ++b)

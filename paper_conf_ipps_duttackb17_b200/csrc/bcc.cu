@@ -531,11 +531,12 @@ ear_status_t cc_run(int32_t nv, const int2 *e, const int32_t *ne, int64_t ne_max
   EAR_LAUNCH(k_iota, grid_for(nv), NT, 0, st)(par, nv);
   for (int it = 0; it < 4 * 32 + 8; ++it) {
     int32_t h = 0;
-    EAR_CUDA_TRY(cudaMemsetAsync(changed, 0, 4, st));
+    EAR_CUDA_TRY(dev_memset(changed, 0, 4, st));
     EAR_LAUNCH(k_cc_hook, grid_for(ne_max), NT, 0, st)(e, ne, par, changed);
     EAR_LAUNCH(k_cc_jump, grid_for(nv), NT, 0, st)(par, nv);
-    EAR_CUDA_TRY(cudaMemcpyAsync(&h, changed, 4, cudaMemcpyDeviceToHost, st));
-    EAR_CUDA_TRY(cudaStreamSynchronize(st));
+    Readback rb(st);
+    EAR_CUDA_TRY(rb.get(&h, changed, 4));
+    EAR_CUDA_TRY(rb.sync());
     if (!h) return EAR_OK;
   }
   set_error("bcc: connected components did not converge");
@@ -585,7 +586,7 @@ ear_status_t bcc_prepare(ear_plan_s *p, int32_t P, cudaStream_t st) {
   }
   b->n_arcs = A;
   int32_t *ne = scal, *changed = scal + 1, *counts = scal + 2, *levels = scal + 6;
-  EAR_CUDA_TRY(cudaMemsetAsync(scal, 0, 32, st));
+  EAR_CUDA_TRY(dev_memset(scal, 0, 32, st));
   const int64_t emax = std::max<int64_t>(A / 2, 1) + nr;
   // 1. connected components
   EAR_LAUNCH(k_edges_all, grid_for(nr), NT, 0, st)(rp, col, nr, e, ne);
@@ -593,32 +594,35 @@ ear_status_t bcc_prepare(ear_plan_s *p, int32_t P, cudaStream_t st) {
   // 2. spanning forest, preorder, low/high
   EAR_LAUNCH(k_tree, 1, TB, 0, st)(nr, rp, col, cc, parent, order, lvl, size, pre, low, high, levels);
   // 3. auxiliary graph -> blocks
-  EAR_CUDA_TRY(cudaMemsetAsync(ne, 0, 4, st));
+  EAR_CUDA_TRY(dev_memset(ne, 0, 4, st));
   EAR_LAUNCH(k_edges_aux, grid_for(nr), NT, 0, st)(rp, col, nr, parent, pre, size, low, high, e, ne);
   EAR_TRY(cc_run(nr, e, ne, emax, blk, changed, st));
-  EAR_CUDA_TRY(cudaMemsetAsync(bcnt, 0, 4 * (size_t)nr, st));
-  EAR_CUDA_TRY(cudaMemsetAsync(ntop, 0, 4 * (size_t)nr, st));
-  EAR_CUDA_TRY(cudaMemsetAsync(rkey, 0, 8 * (size_t)nr, st));
+  EAR_CUDA_TRY(dev_memset(bcnt, 0, 4 * (size_t)nr, st));
+  EAR_CUDA_TRY(dev_memset(ntop, 0, 4 * (size_t)nr, st));
+  EAR_CUDA_TRY(dev_memset(rkey, 0, 8 * (size_t)nr, st));
   EAR_LAUNCH(k_block_stats, grid_for(nr), NT, 0, st)(nr, parent, blk, bcnt, top);
   EAR_LAUNCH(k_root_blocks, grid_for(nr), NT, 0, st)(nr, parent, blk, bcnt, top, cc, rkey, ntop, counts);
   EAR_LAUNCH(k_root_of_comp, grid_for(nr), NT, 0, st)(nr, cc, parent, ntop, rkey, rblock, counts);
   // 4. the remainder graph (edges outside the root blocks) -> hanging pieces and attachments
-  EAR_CUDA_TRY(cudaMemsetAsync(ne, 0, 4, st));
+  EAR_CUDA_TRY(dev_memset(ne, 0, 4, st));
   EAR_LAUNCH(k_edges_rest, grid_for(nr), NT, 0, st)(rp, col, nr, parent, pre, blk, cc, rblock, e, ne);
   EAR_TRY(cc_run(nr, e, ne, emax, rc, changed, st));
-  EAR_CUDA_TRY(cudaMemsetAsync(hsz, 0, 4 * (size_t)nr, st));
+  EAR_CUDA_TRY(dev_memset(hsz, 0, 4 * (size_t)nr, st));
   EAR_LAUNCH(k_attach, grid_for(nr), NT, 0, st)(nr, cc, rblock, blk, top, rc, att_of, hsz);
   // 5. pieces: ids, sizes, layout
   EAR_LAUNCH(k_piece_count, grid_for(nr), NT, 0, st)(nr, cc, rc, hsz, cnt);
   size_t tb = 0, tb2 = 0, tb3 = 0;
   cub::DeviceScan::ExclusiveSum(nullptr, tb, cnt, pid0, nr + 1, st);
   void *tmp = T.get<char>((int64_t)tb);
-  EAR_CUDA_TRY(cudaMemsetAsync(cnt + nr, 0, 4, st));
+  EAR_CUDA_TRY(dev_memset(cnt + nr, 0, 4, st));
   EAR_CUDA_TRY(cub::DeviceScan::ExclusiveSum(tmp, tb, cnt, pid0, nr + 1, st));
   int32_t np = 0, hcounts[8] = {0};
-  EAR_CUDA_TRY(cudaMemcpyAsync(&np, pid0 + nr, 4, cudaMemcpyDeviceToHost, st));
-  EAR_CUDA_TRY(cudaMemcpyAsync(hcounts, scal, 32, cudaMemcpyDeviceToHost, st));
-  EAR_CUDA_TRY(cudaStreamSynchronize(st));
+  {
+    Readback rb(st);
+    EAR_CUDA_TRY(rb.get(&np, pid0 + nr, 4));
+    EAR_CUDA_TRY(rb.get(hcounts, scal, 32));
+    EAR_CUDA_TRY(rb.sync());
+  }
   b->n_blocks = hcounts[2];
   b->n_components = hcounts[3];
   b->n_articulation = hcounts[4];
@@ -632,8 +636,8 @@ ear_status_t bcc_prepare(ear_plan_s *p, int32_t P, cudaStream_t st) {
     set_error("bcc_prepare: out of device memory");
     return EAR_ENOMEM;
   }
-  EAR_CUDA_TRY(cudaMemsetAsync(palloc + np, 0, 8, st));
-  EAR_CUDA_TRY(cudaMemsetAsync(b->psize + np, 0, 4, st));
+  EAR_CUDA_TRY(dev_memset(palloc + np, 0, 8, st));
+  EAR_CUDA_TRY(dev_memset(b->psize + np, 0, 4, st));
   EAR_LAUNCH(k_piece_sizes, grid_for(nr), NT, 0, st)(nr, cc, rc, hsz, rblock, bcnt, pid0, P, b->psize, b->pld, palloc);
   cub::DeviceScan::ExclusiveSum(nullptr, tb2, palloc, b->pbase, np + 1, st);
   cub::DeviceScan::ExclusiveSum(nullptr, tb3, b->psize, pstart, np + 1, st);
@@ -648,8 +652,8 @@ ear_status_t bcc_prepare(ear_plan_s *p, int32_t P, cudaStream_t st) {
   int bits = 1;
   while ((1ll << bits) <= np) ++bits;
   EAR_CUDA_TRY(cub::DeviceRadixSort::SortPairs(tmp2, tbs, keys0, keys1, vals0, vals1, (int)(2 * (int64_t)nr), 0, bits, st));
-  EAR_CUDA_TRY(cudaMemsetAsync(b->ridx, 0xFF, 4 * (size_t)nr, st));
-  EAR_CUDA_TRY(cudaMemsetAsync(hloc, 0xFF, 4 * (size_t)nr, st));
+  EAR_CUDA_TRY(dev_memset(b->ridx, 0xFF, 4 * (size_t)nr, st));
+  EAR_CUDA_TRY(dev_memset(hloc, 0xFF, 4 * (size_t)nr, st));
   EAR_LAUNCH(k_member_local, grid_for(2 * (int64_t)nr), NT, 0, st)(2 * (int64_t)nr, keys1, vals1, pstart, np, cc, pid0,
                                                                   b->ridx, hloc);
   EAR_LAUNCH(k_vertex_info, grid_for(nr), NT, 0, st)(nr, cc, rc, hsz, att_of, pid0, b->ridx, hloc, b->att, b->hp,
@@ -660,10 +664,13 @@ ear_status_t bcc_prepare(ear_plan_s *p, int32_t P, cudaStream_t st) {
   b->h_psize.resize(np);
   b->h_pld.resize(np);
   b->h_pbase.resize(np + 1);
-  EAR_CUDA_TRY(cudaMemcpyAsync(b->h_psize.data(), b->psize, 4 * (size_t)np, cudaMemcpyDeviceToHost, st));
-  EAR_CUDA_TRY(cudaMemcpyAsync(b->h_pld.data(), b->pld, 4 * (size_t)np, cudaMemcpyDeviceToHost, st));
-  EAR_CUDA_TRY(cudaMemcpyAsync(b->h_pbase.data(), b->pbase, 8 * (size_t)(np + 1), cudaMemcpyDeviceToHost, st));
-  EAR_CUDA_TRY(cudaStreamSynchronize(st));
+  {
+    Readback rb(st);
+    EAR_CUDA_TRY(rb.get(b->h_psize.data(), b->psize, 4 * (size_t)np));
+    EAR_CUDA_TRY(rb.get(b->h_pld.data(), b->pld, 4 * (size_t)np));
+    EAR_CUDA_TRY(rb.get(b->h_pbase.data(), b->pbase, 8 * (size_t)(np + 1)));
+    EAR_CUDA_TRY(rb.sync());
+  }
   EAR_CUDA_TRY(cudaGetLastError());
   b->pool_ints = b->h_pbase[np];
   b->largest = 0;
@@ -768,11 +775,14 @@ static ear_status_t piece_rereduce(ear_plan_s *p, ear_bcc_s *b, int32_t id, int3
   int32_t *e = nullptr;
   EAR_CUDA_TRY(cudaMallocAsync((void **)&e, sizeof(int32_t) * (3 * (size_t)A + 1), st));
   int32_t *cnt = e + 3 * (size_t)A;
-  EAR_CUDA_TRY(cudaMemsetAsync(cnt, 0, sizeof(int32_t), st));
+  EAR_CUDA_TRY(dev_memset(cnt, 0, sizeof(int32_t), st));
   EAR_LAUNCH(k_piece_edges, grid_for(A), NT, 0, st)(b->arcs, A, id, e, e + A, e + 2 * (size_t)A, cnt);
   int32_t m = 0;
-  EAR_CUDA_TRY(cudaMemcpyAsync(&m, cnt, sizeof(int32_t), cudaMemcpyDeviceToHost, st));
-  EAR_CUDA_TRY(cudaStreamSynchronize(st));
+  {
+    Readback rb(st);
+    EAR_CUDA_TRY(rb.get(&m, cnt, sizeof(int32_t)));
+    EAR_CUDA_TRY(rb.sync());
+  }
   int32_t levels = 0, n_last = np;
   ear_status_t s = reduce_solve(p, np, m, e, e + A, e + 2 * (size_t)A, M, ld, comm, 0, st, done, &levels, &n_last);
   cudaFreeAsync(e, st);

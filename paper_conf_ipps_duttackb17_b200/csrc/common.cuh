@@ -2,6 +2,7 @@
 #pragma once
 #include <cstdint>
 #include <cstdio>
+#include <vector>
 #include <cuda_runtime.h>
 
 #include "ear_apsp.h"
@@ -94,6 +95,33 @@ void count_launch(int n = 1);
 int prof_begin(int kind, cudaStream_t s);                // -1 when profiling is off
 void prof_end(int slot, cudaStream_t s, double work);
 void prof_fw16_precheck();   // a packed FW abandoned after round 0 by its cap precheck
+// Small device -> host readbacks (counts, flags, piece sizes) that bypass the copy engines: a one-warp
+// kernel stores the bytes into a slot of a mapped pinned staging buffer (thread-local, LIFO slots), so a
+// readback never queues behind a previous job's multi-GB device -> host row copies on the copy engine
+// (apsp_full_host_async pipelining).  get() enqueues on the stream; sync() synchronises the stream and
+// delivers every slot to its destination.  Destroyed without sync(): synchronises, delivers nothing.
+class Readback {
+ public:
+  explicit Readback(cudaStream_t st);
+  ~Readback();
+  Readback(const Readback &) = delete;
+  Readback &operator=(const Readback &) = delete;
+  cudaError_t get(void *h_dst, const void *d_src, size_t bytes);
+  cudaError_t sync();
+
+ private:
+  struct Slot { void *dst; size_t off, bytes; };
+  cudaStream_t st_;
+  size_t base_, used_;
+  bool pending_ = false;
+  std::vector<Slot> slots_;
+};
+// the same store straight into caller-owned pinned (mapped) host memory; completion is the caller's event
+cudaError_t readback_direct(void *h_mapped, const void *d_src, size_t bytes, cudaStream_t st);
+// cudaMemsetAsync / device-to-device cudaMemcpyAsync as SM kernels (prof.cu): the copy engines may be busy
+// for seconds with a previous job's device -> host row copies, and an engine-side memset queues behind them
+cudaError_t dev_memset(void *dst, int value, size_t bytes, cudaStream_t st);
+cudaError_t dev_copy(void *dst, const void *src, size_t bytes, cudaStream_t st);
 // launch one of the library's kernels and count it: EAR_LAUNCH(k, grid, block, smem, stream)(args);
 #define EAR_LAUNCH(k, g, b, sm, st) ::ear::count_launch(), k<<<(g), (b), (sm), (st)>>>
 // decompose.cu

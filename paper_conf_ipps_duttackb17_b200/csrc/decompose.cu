@@ -331,11 +331,14 @@ ear_status_t decompose(int32_t n, int64_t m, const int32_t *src, const int32_t *
   //      must not be processed further, so we sync once here as well -- cheap).
   int32_t *d_flags;
   EAR_TRY(S.alloc(&d_flags, 8));
-  EAR_CUDA_TRY(cudaMemsetAsync(d_flags, 0, sizeof(int32_t) * 8, st));
+  EAR_CUDA_TRY(dev_memset(d_flags, 0, sizeof(int32_t) * 8, st));
   if (m > 0) EAR_LAUNCH(k_validate, grid_for(m), NT, 0, st)(src, dst, w, m, n, d_flags);
   int32_t h_flags[3];
-  EAR_CUDA_TRY(cudaMemcpyAsync(h_flags, d_flags, sizeof(h_flags), cudaMemcpyDeviceToHost, st));
-  EAR_CUDA_TRY(cudaStreamSynchronize(st));
+  {
+    Readback rb(st);
+    EAR_CUDA_TRY(rb.get(h_flags, d_flags, sizeof(h_flags)));
+    EAR_CUDA_TRY(rb.sync());
+  }
   if (h_flags[0]) {
     set_error("ear_decompose: vertex id out of [0,%d) or weight < 1", n);
     return EAR_EINVAL;
@@ -372,8 +375,9 @@ ear_status_t decompose(int32_t n, int64_t m, const int32_t *src, const int32_t *
     EAR_CUDA_TRY(cub::DeviceReduce::ReduceByKey(tmp, tb_red, dk.Current(), ukeys, dv.Current(), uw, d_nruns,
                                                 MinOp(), (int)M2, st));
     int32_t h_runs;
-    EAR_CUDA_TRY(cudaMemcpyAsync(&h_runs, d_nruns, sizeof(int32_t), cudaMemcpyDeviceToHost, st));
-    EAR_CUDA_TRY(cudaStreamSynchronize(st));
+    Readback rbk(st);
+    EAR_CUDA_TRY(rbk.get(&h_runs, d_nruns, sizeof(int32_t)));
+    EAR_CUDA_TRY(rbk.sync());
     A = h_runs - (h_flags[2] > 0 ? 1 : 0);   // drop the self-loop sentinel run
   }
   plan->m_simple = A / 2;
@@ -383,7 +387,7 @@ ear_status_t decompose(int32_t n, int64_t m, const int32_t *src, const int32_t *
   EAR_TRY(S.alloc(&asrc, A)); EAR_TRY(S.alloc(&adst, A));
   EAR_TRY(S.alloc(&deg, n + 1)); EAR_TRY(S.alloc(&rowptr, n + 1));
   EAR_TRY(S.alloc(&term, n)); EAR_TRY(S.alloc(&scan, n + 1));
-  EAR_CUDA_TRY(cudaMemsetAsync(deg, 0, sizeof(int32_t) * (n + 1), st));
+  EAR_CUDA_TRY(dev_memset(deg, 0, sizeof(int32_t) * (n + 1), st));
   if (A > 0) EAR_LAUNCH(k_split_arcs, grid_for(A), NT, 0, st)(ukeys, A, asrc, adst, deg);
   {
     size_t tb = 0;
@@ -412,13 +416,14 @@ ear_status_t decompose(int32_t n, int64_t m, const int32_t *src, const int32_t *
     if (A > 0) EAR_LAUNCH(k_rank_init, grid_for(A), NT, 0, st)(A, asrc, adst, uw, rowptr, term, rb[0]);
     bool cycles = false;
     for (int round = 0; A > 0; ++round) {
-      EAR_CUDA_TRY(cudaMemsetAsync(d_cnt, 0, sizeof(unsigned long long) * 2, st));
+      EAR_CUDA_TRY(dev_memset(d_cnt, 0, sizeof(unsigned long long) * 2, st));
       EAR_LAUNCH(k_rank_round, grid_for(A), NT, 0, st)(A, rb[cur], rb[cur ^ 1], d_cnt);
       cur ^= 1;
       total_rounds++;
       unsigned long long h_cnt[2];
-      EAR_CUDA_TRY(cudaMemcpyAsync(h_cnt, d_cnt, sizeof(h_cnt), cudaMemcpyDeviceToHost, st));
-      EAR_CUDA_TRY(cudaStreamSynchronize(st));
+      Readback rbk(st);
+      EAR_CUDA_TRY(rbk.get(h_cnt, d_cnt, sizeof(h_cnt)));
+      EAR_CUDA_TRY(rbk.sync());
       if (h_cnt[1] == 0) break;                      // every arc ranked
       if (h_cnt[0] == 0) { cycles = true; break; }   // only pure-cycle arcs remain (C5)
     }
@@ -434,13 +439,14 @@ ear_status_t decompose(int32_t n, int64_t m, const int32_t *src, const int32_t *
     EAR_LAUNCH(k_cycle_init, grid_for(A), NT, 0, st)(A, rb[cur].done, asrc, adst, rowptr, lab[0], cn[0]);
     int c = 0;
     for (;;) {
-      EAR_CUDA_TRY(cudaMemsetAsync(d_changed, 0, sizeof(int32_t), st));
+      EAR_CUDA_TRY(dev_memset(d_changed, 0, sizeof(int32_t), st));
       EAR_LAUNCH(k_cycle_round, grid_for(A), NT, 0, st)(A, rb[cur].done, lab[c], cn[c], lab[c ^ 1], cn[c ^ 1], d_changed);
       c ^= 1;
       total_rounds++;
       int32_t h_changed;
-      EAR_CUDA_TRY(cudaMemcpyAsync(&h_changed, d_changed, sizeof(int32_t), cudaMemcpyDeviceToHost, st));
-      EAR_CUDA_TRY(cudaStreamSynchronize(st));
+      Readback rbk(st);
+      EAR_CUDA_TRY(rbk.get(&h_changed, d_changed, sizeof(int32_t)));
+      EAR_CUDA_TRY(rbk.sync());
       if (!h_changed) break;
     }
     EAR_LAUNCH(k_cycle_promote, grid_for(A), NT, 0, st)(A, rb[cur].done, asrc, lab[c], term);
@@ -457,8 +463,9 @@ ear_status_t decompose(int32_t n, int64_t m, const int32_t *src, const int32_t *
     EAR_CUDA_TRY(cub::DeviceScan::ExclusiveSum(tmp, tb, term, scan, n, st));
   }
   int32_t h_last[2];
-  EAR_CUDA_TRY(cudaMemcpyAsync(&h_last[0], scan + n - 1, sizeof(int32_t), cudaMemcpyDeviceToHost, st));
-  EAR_CUDA_TRY(cudaMemcpyAsync(&h_last[1], term + n - 1, sizeof(int32_t), cudaMemcpyDeviceToHost, st));
+  Readback rbk(st);   // delivered at the N_r synchronisation point below
+  EAR_CUDA_TRY(rbk.get(&h_last[0], scan + n - 1, sizeof(int32_t)));
+  EAR_CUDA_TRY(rbk.get(&h_last[1], term + n - 1, sizeof(int32_t)));
 
   // descriptors
   EAR_TRY(plan_alloc(&plan->desc, n, st));
@@ -471,8 +478,8 @@ ear_status_t decompose(int32_t n, int64_t m, const int32_t *src, const int32_t *
   EAR_TRY(S.alloc(&ear_cnt, A)); EAR_TRY(S.alloc(&d_stats, 2));
   EAR_TRY(S.alloc(&seg_key, n)); EAR_TRY(S.alloc(&seg_key2, n));
   EAR_TRY(S.alloc(&seg_val, n)); EAR_TRY(S.alloc(&seg_val2, n));
-  EAR_CUDA_TRY(cudaMemsetAsync(ear_cnt, 0, sizeof(int32_t) * std::max<int64_t>(A, 1), st));
-  EAR_CUDA_TRY(cudaMemsetAsync(d_stats, 0, sizeof(int32_t) * 2, st));
+  EAR_CUDA_TRY(dev_memset(ear_cnt, 0, sizeof(int32_t) * std::max<int64_t>(A, 1), st));
+  EAR_CUDA_TRY(dev_memset(d_stats, 0, sizeof(int32_t) * 2, st));
   const uint64_t seg_sentinel = (uint64_t)(uint32_t)std::max<int64_t>(A, 1) << 32;
   EAR_LAUNCH(k_descriptors, grid_for(n), NT, 0, st)(n, term, scan, rowptr, rb[cur], plan->desc, plan->tid, plan->ear,
                                             ear_cnt, seg_key, seg_val, seg_sentinel);
@@ -481,13 +488,13 @@ ear_status_t decompose(int32_t n, int64_t m, const int32_t *src, const int32_t *
   // reduced arcs: count, then emit
   unsigned long long *d_rcount;
   EAR_TRY(S.alloc(&d_rcount, 1));
-  EAR_CUDA_TRY(cudaMemsetAsync(d_rcount, 0, sizeof(unsigned long long), st));
+  EAR_CUDA_TRY(dev_memset(d_rcount, 0, sizeof(unsigned long long), st));
   if (A > 0) EAR_LAUNCH(k_reduced_arcs, grid_for(A), NT, 0, st)(A, asrc, term, scan, rb[cur], nullptr, nullptr, nullptr, d_rcount, 0);
   unsigned long long h_rcount = 0;
   int32_t h_stats[2];
-  EAR_CUDA_TRY(cudaMemcpyAsync(&h_rcount, d_rcount, sizeof(h_rcount), cudaMemcpyDeviceToHost, st));
-  EAR_CUDA_TRY(cudaMemcpyAsync(h_stats, d_stats, sizeof(h_stats), cudaMemcpyDeviceToHost, st));
-  EAR_CUDA_TRY(cudaStreamSynchronize(st));
+  EAR_CUDA_TRY(rbk.get(&h_rcount, d_rcount, sizeof(h_rcount)));
+  EAR_CUDA_TRY(rbk.get(h_stats, d_stats, sizeof(h_stats)));
+  EAR_CUDA_TRY(rbk.sync());
   plan->n_reduced = h_last[0] + h_last[1];
   plan->n_chains = h_stats[0];
   plan->max_chain_len = h_stats[1];
@@ -495,7 +502,7 @@ ear_status_t decompose(int32_t n, int64_t m, const int32_t *src, const int32_t *
   EAR_TRY(plan_alloc(&plan->re_u, plan->n_redges, st));
   EAR_TRY(plan_alloc(&plan->re_v, plan->n_redges, st));
   EAR_TRY(plan_alloc(&plan->re_w, plan->n_redges, st));
-  EAR_CUDA_TRY(cudaMemsetAsync(d_rcount, 0, sizeof(unsigned long long), st));
+  EAR_CUDA_TRY(dev_memset(d_rcount, 0, sizeof(unsigned long long), st));
   if (A > 0)
     EAR_LAUNCH(k_reduced_arcs, grid_for(A), NT, 0, st)(A, asrc, term, scan, rb[cur], plan->re_u, plan->re_v, plan->re_w,
                                               d_rcount, 1);
@@ -532,12 +539,12 @@ ear_status_t decompose(int32_t n, int64_t m, const int32_t *src, const int32_t *
   }
   if (plan->n_promoted < 0) {
     // promoted pure-cycle anchors = terminals of degree two (C5)
-    EAR_CUDA_TRY(cudaMemsetAsync(d_stats, 0, sizeof(int32_t), st));
+    EAR_CUDA_TRY(dev_memset(d_stats, 0, sizeof(int32_t), st));
     EAR_LAUNCH(k_count_promoted, grid_for(n), NT, 0, st)(n, deg, term, d_stats);
-    EAR_CUDA_TRY(cudaMemcpyAsync(h_stats, d_stats, sizeof(int32_t), cudaMemcpyDeviceToHost, st));
+    EAR_CUDA_TRY(rbk.get(h_stats, d_stats, sizeof(int32_t)));
   }
   EAR_CUDA_TRY(cudaGetLastError());
-  EAR_CUDA_TRY(cudaStreamSynchronize(st));
+  EAR_CUDA_TRY(rbk.sync());
   if (plan->n_promoted < 0) plan->n_promoted = h_stats[0];
   return EAR_OK;
 }

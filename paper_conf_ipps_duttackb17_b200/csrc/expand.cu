@@ -320,7 +320,7 @@ ear_status_t expand(const ear_plan_s *plan, const int32_t *D, int64_t ldd, int32
     W.n_items = groups * W.segmajor;
   }
   EAR_CUDA_TRY(cudaMallocAsync((void **)&W.counter, sizeof(int32_t), st));
-  EAR_CUDA_TRY(cudaMemsetAsync(W.counter, 0, sizeof(int32_t), st));
+  EAR_CUDA_TRY(dev_memset(W.counter, 0, sizeof(int32_t), st));
   const unsigned grid = (unsigned)std::min<int64_t>(W.n_items, slots);
   const double nr = plan->n_reduced;
   int se = prof_begin(prof_kind, st);

@@ -1349,7 +1349,8 @@ struct Precheck {
   bool on = false;
   static int32_t *host() {   // pinned, one per process (one FW at a time)
     static int32_t *h = nullptr;
-    if (!h && cudaMallocHost((void **)&h, sizeof(int32_t)) != cudaSuccess) h = nullptr;
+    if (!h && cudaHostAlloc((void **)&h, sizeof(int32_t), cudaHostAllocMapped | cudaHostAllocPortable) != cudaSuccess)
+      h = nullptr;
     return h;
   }
   void start(ear_plan_s *plan, int32_t Np, int32_t n_real, int nt) {
@@ -1357,11 +1358,11 @@ struct Precheck {
     on = cudaStreamCreateWithFlags(&hs, cudaStreamNonBlocking) == cudaSuccess &&
          cudaEventCreateWithFlags(&ev, cudaEventDisableTiming) == cudaSuccess &&
          cudaMallocAsync((void **)&row, sizeof(int32_t) * ((size_t)Np + 1), hs) == cudaSuccess &&
-         cudaMemsetAsync(row + Np, 0, sizeof(int32_t), hs) == cudaSuccess &&
+         dev_memset(row + Np, 0, sizeof(int32_t), hs) == cudaSuccess &&
          sssp_rows(plan, row, Np, Np, 0, 1, nullptr, hs) == EAR_OK;
     if (on) {
       EAR_LAUNCH(k_row_far, grid_for(n_real), 256, 0, hs)(row, n_real, row + Np);
-      on = cudaMemcpyAsync(host(), row + Np, sizeof(int32_t), cudaMemcpyDeviceToHost, hs) == cudaSuccess &&
+      on = readback_direct(host(), row + Np, sizeof(int32_t), hs) == cudaSuccess &&
            cudaEventRecord(ev, hs) == cudaSuccess;
     }
     if (!on) cudaGetLastError();
@@ -1493,11 +1494,12 @@ ear_status_t fw_single16(int32_t *D, int64_t ldd, int32_t Np, const int32_t *lab
   if (s == EAR_OK && hopeless) prof_fw16_precheck();
   if (s == EAR_OK && !hopeless) {
     int sc = prof_begin(PK_FW16_CONV, st);
-    cudaMemsetAsync(bad, 0, sizeof(int32_t), st);
+    dev_memset(bad, 0, sizeof(int32_t), st);
     EAR_LAUNCH(k_check16, grid_for((int64_t)Np * (Np / 8)), 256, 0, st)(D16, Np, lab, n_real, bad);
     prof_end(sc, st, 0);
-    cudaError_t e = cudaMemcpyAsync(&h_bad, bad, sizeof(int32_t), cudaMemcpyDeviceToHost, st);
-    if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+    Readback rb(st);
+    cudaError_t e = rb.get(&h_bad, bad, sizeof(int32_t));
+    if (e == cudaSuccess) e = rb.sync();
     if (e != cudaSuccess) { set_error("fw_single16: %s", cudaGetErrorString(e)); s = EAR_ECUDA; }
   }
   if (s == EAR_OK && h_bad == 0) {
@@ -1913,15 +1915,16 @@ static ear_status_t fw_sharded16(std::vector<Shard *> &sh, int32_t Np, ear_comm_
   }
   if (s == EAR_OK) {
     int sc = prof_begin(PK_FW16_CONV, st);
-    cudaMemsetAsync(flag, 0, sizeof(int32_t), st);
+    dev_memset(flag, 0, sizeof(int32_t), st);
     for (size_t r = 0; r < R; ++r)
       if (sh[r]->nown > 0)
         EAR_LAUNCH(k_check16_list, grid_for((int64_t)sh[r]->nown * TILE * (Np / 8)), 256, 0, st)(
             S16[r], Np, sh[r]->d_rows, sh[r]->nown, Np, lab, n_real, flag);
     prof_end(sc, st, 0);
     if (comm) s = comm_allreduce_min(comm, flag, 1, st);
-    cudaError_t e = cudaMemcpyAsync(&h_flag, flag, sizeof(int32_t), cudaMemcpyDeviceToHost, st);
-    if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+    Readback rb(st);
+    cudaError_t e = rb.get(&h_flag, flag, sizeof(int32_t));
+    if (e == cudaSuccess) e = rb.sync();
     if (s == EAR_OK && e != cudaSuccess) { set_error("fw_sharded16: %s", cudaGetErrorString(e)); s = EAR_ECUDA; }
   }
   if (s == EAR_OK && h_flag == 0) {
@@ -2086,11 +2089,12 @@ ear_status_t reduced_labels(ear_plan_s *p, int32_t Np, cudaStream_t st, const in
     for (int it = 0; it < 64 && s == EAR_OK; ++it) {
       int32_t h = 0;
       if (p->n_redges == 0) break;
-      cudaMemsetAsync(changed, 0, sizeof(int32_t), st);
+      dev_memset(changed, 0, sizeof(int32_t), st);
       EAR_LAUNCH(k_cc_hook16, grid_for(p->n_redges), 256, 0, st)(p->re_u, p->re_v, p->n_redges, p->cc, changed);
       EAR_LAUNCH(k_cc_jump16, grid_for(Np), 256, 0, st)(p->cc, Np);
-      cudaError_t e = cudaMemcpyAsync(&h, changed, sizeof(int32_t), cudaMemcpyDeviceToHost, st);
-      if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+      Readback rb(st);
+      cudaError_t e = rb.get(&h, changed, sizeof(int32_t));
+      if (e == cudaSuccess) e = rb.sync();
       if (e != cudaSuccess) { set_error("reduced_labels: %s", cudaGetErrorString(e)); s = EAR_ECUDA; }
       if (!h) break;
     }

@@ -1,5 +1,7 @@
 // Launch counting and optional CUDA-event profiling of the library's kernels (ear_profile_* ABI).
+#include <algorithm>
 #include <atomic>
+#include <cstring>
 #include <mutex>
 #include <vector>
 
@@ -62,6 +64,115 @@ void prof_end(int slot, cudaStream_t s, double work) {
   if (slot >= (int)g_pending.size()) return;
   g_pending[slot].work = work;
   cudaEventRecord(g_pending[slot].e1, s);
+}
+
+
+// ---- small readbacks through mapped pinned memory (see Readback in common.cuh)
+namespace {
+constexpr size_t kStageBytes = 1 << 20;
+struct Stage {
+  char *h = nullptr;   // mapped pinned; the same pointer is valid on the device (UVA)
+  size_t used = 0;
+  bool failed = false;
+};
+thread_local Stage t_stage;
+
+__global__ void k_readback(const unsigned char *__restrict__ src, unsigned char *__restrict__ dst, size_t bytes) {
+  const bool w4 = ((reinterpret_cast<uintptr_t>(src) | reinterpret_cast<uintptr_t>(dst) | bytes) & 3) == 0;
+  if (w4) {
+    const uint32_t *s = reinterpret_cast<const uint32_t *>(src);
+    uint32_t *d = reinterpret_cast<uint32_t *>(dst);
+    for (size_t i = blockIdx.x * blockDim.x + threadIdx.x; i < bytes / 4; i += (size_t)gridDim.x * blockDim.x) d[i] = s[i];
+  } else {
+    for (size_t i = blockIdx.x * blockDim.x + threadIdx.x; i < bytes; i += (size_t)gridDim.x * blockDim.x) dst[i] = src[i];
+  }
+}
+
+cudaError_t launch_readback(void *dst, const void *src, size_t bytes, cudaStream_t st) {
+  const int grid = (int)std::min<size_t>(64, (bytes / 4 + 255) / 256 + 1);
+  EAR_LAUNCH(k_readback, grid, 256, 0, st)(static_cast<const unsigned char *>(src), static_cast<unsigned char *>(dst), bytes);
+  return cudaGetLastError();
+}
+}  // namespace
+
+namespace {
+__global__ void k_fill(unsigned char *__restrict__ dst, uint32_t word, size_t bytes) {
+  const size_t stride = (size_t)gridDim.x * blockDim.x, t0 = blockIdx.x * (size_t)blockDim.x + threadIdx.x;
+  const size_t mis = (16 - (reinterpret_cast<uintptr_t>(dst) & 15)) & 15, head = mis < bytes ? mis : bytes;
+  for (size_t i = t0; i < head; i += stride) dst[i] = (unsigned char)word;
+  uint4 *v = reinterpret_cast<uint4 *>(dst + head);
+  const size_t nv = (bytes - head) / 16;
+  for (size_t i = t0; i < nv; i += stride) v[i] = make_uint4(word, word, word, word);
+  for (size_t i = head + nv * 16 + t0; i < bytes; i += stride) dst[i] = (unsigned char)word;
+}
+__global__ void k_copy_bytes(unsigned char *__restrict__ dst, const unsigned char *__restrict__ src, size_t bytes) {
+  const size_t stride = (size_t)gridDim.x * blockDim.x, t0 = blockIdx.x * (size_t)blockDim.x + threadIdx.x;
+  if (((reinterpret_cast<uintptr_t>(dst) | reinterpret_cast<uintptr_t>(src)) & 15) == 0) {
+    const size_t nv = bytes / 16;
+    for (size_t i = t0; i < nv; i += stride) reinterpret_cast<uint4 *>(dst)[i] = reinterpret_cast<const uint4 *>(src)[i];
+    for (size_t i = nv * 16 + t0; i < bytes; i += stride) dst[i] = src[i];
+  } else {
+    for (size_t i = t0; i < bytes; i += stride) dst[i] = src[i];
+  }
+}
+int fill_grid(size_t bytes) { return (int)std::max<size_t>(1, std::min<size_t>(148 * 8, (bytes / 16 + 255) / 256)); }
+}  // namespace
+
+cudaError_t dev_memset(void *dst, int value, size_t bytes, cudaStream_t st) {
+  if (!bytes) return cudaSuccess;
+  const uint32_t b = (uint32_t)(value & 0xFF);
+  EAR_LAUNCH(k_fill, fill_grid(bytes), 256, 0, st)(static_cast<unsigned char *>(dst), b * 0x01010101u, bytes);
+  return cudaGetLastError();
+}
+
+cudaError_t dev_copy(void *dst, const void *src, size_t bytes, cudaStream_t st) {
+  if (!bytes) return cudaSuccess;
+  EAR_LAUNCH(k_copy_bytes, fill_grid(bytes), 256, 0, st)(static_cast<unsigned char *>(dst),
+                                                         static_cast<const unsigned char *>(src), bytes);
+  return cudaGetLastError();
+}
+
+Readback::Readback(cudaStream_t st) : st_(st) {
+  Stage &g = t_stage;
+  if (!g.h && !g.failed && cudaHostAlloc((void **)&g.h, kStageBytes, cudaHostAllocMapped | cudaHostAllocPortable) != cudaSuccess) {
+    cudaGetLastError();
+    g.h = nullptr;
+    g.failed = true;
+  }
+  base_ = used_ = g.used;
+}
+
+Readback::~Readback() {
+  if (pending_) cudaStreamSynchronize(st_);   // error path: let the stores land before the slots are reused
+  t_stage.used = base_;
+}
+
+cudaError_t Readback::get(void *h_dst, const void *d_src, size_t bytes) {
+  if (bytes == 0) return cudaSuccess;
+  Stage &g = t_stage;
+  const size_t off = (used_ + 15) & ~size_t(15);
+  pending_ = true;
+  if (!g.h || off + bytes > kStageBytes)   // no staging (or too big): the plain copy
+    return cudaMemcpyAsync(h_dst, d_src, bytes, cudaMemcpyDeviceToHost, st_);
+  cudaError_t e = launch_readback(g.h + off, d_src, bytes, st_);
+  if (e != cudaSuccess) return e;
+  slots_.push_back({h_dst, off, bytes});
+  used_ = g.used = off + bytes;
+  return cudaSuccess;
+}
+
+cudaError_t Readback::sync() {
+  cudaError_t e = cudaStreamSynchronize(st_);
+  pending_ = false;
+  if (e == cudaSuccess)
+    for (const Slot &s : slots_) std::memcpy(s.dst, t_stage.h + s.off, s.bytes);
+  slots_.clear();
+  used_ = t_stage.used = base_;
+  return e;
+}
+
+cudaError_t readback_direct(void *h_mapped, const void *d_src, size_t bytes, cudaStream_t st) {
+  return bytes ? launch_readback(h_mapped, d_src, bytes, st) : cudaSuccess;
 }
 
 }  // namespace ear

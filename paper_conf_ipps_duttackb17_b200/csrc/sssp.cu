@@ -442,20 +442,21 @@ ear_status_t sssp_prepare(ear_plan_s *p, cudaStream_t st) {
     EAR_CUDA_TRY(cub::DeviceRadixSort::SortPairs(tmp, tb1, dk, dv, (int)E, 0, 32 + bits, st));
     EAR_CUDA_TRY(cub::DeviceReduce::ReduceByKey(tmp, tb2, dk.Current(), uk, dv.Current(), uv, nruns, MinOp(), (int)E,
                                                 st));
-    EAR_CUDA_TRY(cudaMemcpyAsync(&A, nruns, 4, cudaMemcpyDeviceToHost, st));
-    EAR_CUDA_TRY(cudaStreamSynchronize(st));
+    Readback rb(st);
+    EAR_CUDA_TRY(rb.get(&A, nruns, 4));
+    EAR_CUDA_TRY(rb.sync());
   }
   EAR_CUDA_TRY(cudaMallocAsync((void **)&p->r_rowptr, 4 * ((size_t)nr + 1), st));
   EAR_CUDA_TRY(cudaMallocAsync((void **)&p->r_col, 4 * (size_t)std::max(A, 1), st));
   EAR_CUDA_TRY(cudaMallocAsync((void **)&p->r_w, 4 * (size_t)std::max(A, 1), st));
-  EAR_CUDA_TRY(cudaMemsetAsync(deg, 0, 4 * ((size_t)nr + 1), st));
+  EAR_CUDA_TRY(dev_memset(deg, 0, 4 * ((size_t)nr + 1), st));
   if (A > 0) {
     const int g = (int)std::min<int64_t>(ceil_div(A, 256), 4096);
     EAR_LAUNCH(k_r_split, g, 256, 0, st)(uk, A, p->r_col, deg);
-    EAR_CUDA_TRY(cudaMemcpyAsync(p->r_w, uv, 4 * (size_t)A, cudaMemcpyDeviceToDevice, st));
+    EAR_CUDA_TRY(dev_copy(p->r_w, uv, 4 * (size_t)A, st));
     EAR_CUDA_TRY(cub::DeviceScan::ExclusiveSum(tmp, tb3, deg, p->r_rowptr, nr + 1, st));
   } else {
-    EAR_CUDA_TRY(cudaMemsetAsync(p->r_rowptr, 0, 4 * ((size_t)nr + 1), st));
+    EAR_CUDA_TRY(dev_memset(p->r_rowptr, 0, 4 * ((size_t)nr + 1), st));
   }
   p->n_rarcs = A;
   void *fr[] = {k0, k1, uk, v0, v1, uv, nruns, deg, tmp};
@@ -534,7 +535,7 @@ ear_status_t sssp_rows(ear_plan_s *p, int32_t *D, int64_t ldd, int32_t Np, int32
   static unsigned long long *d_stats = nullptr;
   static const bool want_stats = getenv("EAR_SSSP_STATS") != nullptr;
   if (want_stats && !d_stats) EAR_CUDA_TRY(cudaMalloc((void **)&d_stats, 32));
-  if (want_stats) EAR_CUDA_TRY(cudaMemsetAsync(d_stats, 0, 32, st));
+  if (want_stats) EAR_CUDA_TRY(dev_memset(d_stats, 0, 32, st));
   int dev = 0, nsm = 148;
   EAR_CUDA_TRY(cudaGetDevice(&dev));
   EAR_CUDA_TRY(cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev));
@@ -546,11 +547,14 @@ ear_status_t sssp_rows(ear_plan_s *p, int32_t *D, int64_t ldd, int32_t Np, int32
     if (!p->r_arcs) {
       int32_t *d_md = nullptr, md = 0;
       EAR_CUDA_TRY(cudaMallocAsync((void **)&d_md, 4, st));
-      EAR_CUDA_TRY(cudaMemsetAsync(d_md, 0, 4, st));
+      EAR_CUDA_TRY(dev_memset(d_md, 0, 4, st));
       EAR_LAUNCH(k_max_deg, (int)std::min<int64_t>(ceil_div(p->n_reduced, 256), 4096), 256, 0, st)(
           p->r_rowptr, p->n_reduced, d_md);
-      EAR_CUDA_TRY(cudaMemcpyAsync(&md, d_md, 4, cudaMemcpyDeviceToHost, st));
-      EAR_CUDA_TRY(cudaStreamSynchronize(st));
+      {
+        Readback rb(st);
+        EAR_CUDA_TRY(rb.get(&md, d_md, 4));
+        EAR_CUDA_TRY(rb.sync());
+      }
       cudaFreeAsync(d_md, st);
       p->r_ell_k = md <= 4 ? 4 : md <= 8 ? 8 : md <= 12 ? 12 : md <= 16 ? 16 : 0;
       if (p->r_ell_k > 0) {
