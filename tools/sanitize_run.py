@@ -1,7 +1,8 @@
 """Small end-to-end runs for compute-sanitizer (memcheck / racecheck / synccheck): every kernel of the
 library on graphs small enough for the instrumented run -- packed and int32 FW (single + emulated
 sharding with the owner-side phase 2 and lookahead), blocks with a re-reduced piece, SSSP, expansion
-(aligned and scalar store paths), query mode, Phase I with pure cycles."""
+(aligned and scalar store paths), query mode, Phase I with pure cycles, the host-buffer entry points
+(two async jobs in flight, pinned and pageable inputs)."""
 import sys
 
 import numpy as np
@@ -26,5 +27,13 @@ for g in [gg.corner_cases(5, n_target=300), gg.torus(12, 12, 150, seed=1), gg.cy
     ea.expand_ears(plan, D, 0, g.n, out=big[:, 1:1 + g.n])
     s = dev(np.arange(g.n)); t = dev(np.arange(g.n)[::-1].copy())
     ea.query_pairs(plan, D, s, t)
+# host-buffer entry points, two async jobs in flight (mapped-pinned readbacks, kernel memsets)
+g = gg.corner_cases(5, n_target=300)
+hs, hd, hw = (torch.as_tensor(np.ascontiguousarray(a, dtype=np.int32)).pin_memory() for a in (g.src, g.dst, g.w))
+outs = [torch.empty((g.n, g.n), dtype=torch.int32, pin_memory=True) for _ in range(2)]
+j0 = ea.apsp_full_host_async(g.n, hs, hd, hw, out=outs[0], flags=ea.FLAG_BCC)
+j1 = ea.apsp_full_host_async(g.n, hs, hd, hw, out=outs[1], flags=ea.FLAG_BCC)
+j0.wait(); j1.wait()
+ea.apsp_full_host(g.n, g.src, g.dst, g.w)   # pageable inputs: the copy-in branch
 torch.cuda.synchronize()
 print("sanitize run ok")
