@@ -95,10 +95,10 @@ void count_launch(int n = 1);
 int prof_begin(int kind, cudaStream_t s);                // -1 when profiling is off
 void prof_end(int slot, cudaStream_t s, double work);
 void prof_fw16_precheck();   // a packed FW abandoned after round 0 by its cap precheck
-// Small device -> host readbacks (counts, flags, piece sizes) that bypass the copy engines: a one-warp
-// kernel stores the bytes into a slot of a mapped pinned staging buffer (thread-local, LIFO slots), so a
-// readback never queues behind a previous job's multi-GB device -> host row copies on the copy engine
-// (apsp_full_host_async pipelining).  get() enqueues on the stream; sync() synchronises the stream and
+// Small device -> host readbacks (counts, flags, piece sizes) that bypass the copy engines: a small
+// kernel stores the bytes into a slot of a mapped pinned staging buffer (1 MB per thread; a get() takes
+// slots above every live object's), so a readback never queues behind a previous job's multi-GB
+// device -> host row copies on the copy engine (apsp_full_host_async pipelining).  get() enqueues on the stream; sync() synchronises the stream and
 // delivers every slot to its destination.  Destroyed without sync(): synchronises, delivers nothing.
 class Readback {
  public:

@@ -144,13 +144,13 @@ Readback::Readback(cudaStream_t st) : st_(st) {
 
 Readback::~Readback() {
   if (pending_) cudaStreamSynchronize(st_);   // error path: let the stores land before the slots are reused
-  t_stage.used = base_;
+  if (t_stage.used == used_) t_stage.used = base_;   // release only when this object holds the top slots
 }
 
 cudaError_t Readback::get(void *h_dst, const void *d_src, size_t bytes) {
   if (bytes == 0) return cudaSuccess;
   Stage &g = t_stage;
-  const size_t off = (used_ + 15) & ~size_t(15);
+  const size_t off = (std::max(used_, g.used) + 15) & ~size_t(15);   // above every live object's slots
   pending_ = true;
   if (!g.h || off + bytes > kStageBytes)   // no staging (or too big): the plain copy
     return cudaMemcpyAsync(h_dst, d_src, bytes, cudaMemcpyDeviceToHost, st_);
@@ -167,7 +167,8 @@ cudaError_t Readback::sync() {
   if (e == cudaSuccess)
     for (const Slot &s : slots_) std::memcpy(s.dst, t_stage.h + s.off, s.bytes);
   slots_.clear();
-  used_ = t_stage.used = base_;
+  if (t_stage.used == used_) t_stage.used = base_;
+  used_ = base_;
   return e;
 }
 
