@@ -377,7 +377,7 @@ def run_ours(args, rank, world, local_rank):
         out_bytes = 4 * rows * g.n
         pipelined = args.e2e_mode == "pipelined"
         # two pinned output buffers when the host has room (job i+1 never lands in job i's rows)
-        nbuf = 2 if pipelined and psutil.virtual_memory().available > 2.5 * out_bytes else 1
+        nbuf = args.e2e_bufs or (2 if pipelined and psutil.virtual_memory().available > 2.5 * out_bytes else 1)
         houts = [torch.empty((rows, g.n), dtype=torch.int32, pin_memory=True) for _ in range(nbuf)]
         ea.apsp_full_host(g.n, hs, hd, hw, out=houts[0], row_begin=r0, row_end=r1, flags=flags, comm=comm,
                           stream=stream)
@@ -452,6 +452,8 @@ def main():
     ap.add_argument("--fw32", action="store_true", help="int32 FW throughout (EAR_FLAG_FW32)")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=4)
+    ap.add_argument("--e2e-bufs", type=int, choices=[0, 1, 2], default=0,
+                    help="pinned host output buffers for the pipelined e2e (0: two when the host has room)")
     ap.add_argument("--e2e-mode", choices=["sync", "pipelined"], default="pipelined",
                     help="e2e calls: synchronous apsp_full_host, or async jobs pipelined one deep")
     ap.add_argument("--no-cpu-baseline", action="store_true")

@@ -212,6 +212,40 @@ def test_host_async_pipelined(pkg, flags):
     assert_exact(shared.numpy(), r1, "async shared buffer")
 
 
+@pytest.mark.parametrize("flags", [0, "bcc"])
+def test_concurrent_host_threads(pkg, flags):
+    """Two host threads, each on its own stream, solving different graphs at the same time: the
+    library's per-thread readback staging and its kernel memsets must not mix the two problems."""
+    import threading
+    fl = pkg.FLAG_BCC if flags == "bcc" else 0
+    gs = [gg.corner_cases(91, n_target=700), gg.torus(10, 14, 120, seed=4), gg.cycle(300, seed=5),
+          gg.config("cfg1")]
+    refs = [oracle.apsp(g.n, g.src, g.dst, g.w) for g in gs]
+    got = [None] * len(gs)
+    errs = []
+
+    def work(k):
+        try:
+            st = torch.cuda.Stream()
+            with torch.cuda.stream(st):
+                for i in range(k, len(gs), 2):
+                    g = gs[i]
+                    out = pkg.apsp_full(g.n, dev(g.src), dev(g.dst), dev(g.w), flags=fl, stream=st)
+                    st.synchronize()
+                    got[i] = out.cpu().numpy()
+        except Exception as e:  # noqa: BLE001  (reported below)
+            errs.append(e)
+
+    ts = [threading.Thread(target=work, args=(k,)) for k in range(2)]
+    for t in ts:
+        t.start()
+    for t in ts:
+        t.join()
+    assert not errs, errs
+    for i, (a, r) in enumerate(zip(got, refs)):
+        assert_exact(a, r, f"thread graph {i}")
+
+
 # ------------------------------------------------------------------------------ degenerate inputs
 def graph(n, edges):
     from paper_conf_ipps_duttackb17_b200.graphgen import Graph
