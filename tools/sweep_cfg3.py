@@ -1,6 +1,7 @@
 #!/usr/bin/env python
 """cfg3 (BASELINE.json configs[2]): 50k-vertex tori with degree-two fraction f = 0/20/40/60/80 %,
-ear-reduced APSP vs direct blocked FW on the whole graph (EAR_FLAG_NO_CONTRACT), one B200.
+ear-reduced APSP (plain FW and Phase II by blocks) vs direct blocked FW on the whole graph
+(EAR_FLAG_NO_CONTRACT), one B200.
 
 For every f: one warm-up + one timed apsp_full per variant (CUDA events), the two 10 GB outputs
 compared bit for bit on the device (pin P7), and the FW min-plus rate.  Prints one JSON line per f
@@ -52,14 +53,19 @@ def main():
         out_d = torch.empty((g.n, g.n), dtype=torch.int32, device="cuda")
         ms_d, pd = timed(lambda: ea.apsp_full(g.n, src, dst, w, out=out_d, flags=ea.FLAG_NO_CONTRACT))
         same = bool(torch.equal(out_r, out_d))
-        del out_r, out_d
+        del out_d
+        out_b = torch.empty((g.n, g.n), dtype=torch.int32, device="cuda")
+        ms_b, _ = timed(lambda: ea.apsp_full(g.n, src, dst, w, out=out_b, flags=ea.FLAG_BCC))
+        same_b = bool(torch.equal(out_r, out_b))
+        del out_r, out_b
         torch.cuda.empty_cache()
         rec = {"config": f"cfg3_f{f}", "n": g.n, "m": g.m, "deg2_frac": st["deg2_frac"], "n_reduced": nr,
                "ear_reduced_ms": ms_r, "direct_fw_ms": ms_d, "speedup": ms_d / ms_r,
                "ear_entries_per_s": g.n * g.n / (ms_r / 1e3), "direct_entries_per_s": g.n * g.n / (ms_d / 1e3),
                "ear_fw_phase3_tminplus": pr["fw_phase3_minplus"] / (pr["fw_phase3_ms"] / 1e3) / 1e12,
                "direct_fw_phase3_tminplus": pd["fw_phase3_minplus"] / (pd["fw_phase3_ms"] / 1e3) / 1e12,
-               "ear_expand_ms": pr["expand_ms"], "bitwise_equal": same}
+               "ear_expand_ms": pr["expand_ms"], "bitwise_equal": same,
+               "ear_bcc_ms": ms_b, "bcc_speedup": ms_d / ms_b, "bcc_bitwise_equal": same_b}
         print(json.dumps(rec), flush=True)
         lines.append(rec)
     if args.out:
