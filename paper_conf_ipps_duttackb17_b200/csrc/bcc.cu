@@ -149,27 +149,42 @@ __global__ void k_edges_rest(const int32_t *rp, const int32_t *col, int32_t nr, 
   }
 }
 
+// ------------------------------------------------------------------ BFS root per component
+// The level sweeps of k_tree cost one barrier-separated step per BFS level, so the root should be central:
+// with spatially coherent labels the min-id vertex (the component label) sits at a corner and the BFS
+// depth is the hop diameter.  Heuristic (any root gives the same blocks): the vertex whose id is closest
+// to the middle of the component's id range [cc, max id].
+__global__ void k_comp_maxid(int32_t nr, const int32_t *cc, int32_t *cmax) { GS(v, nr) atomicMax(&cmax[cc[v]], (int32_t)v); }
+__global__ void k_comp_root(int32_t nr, const int32_t *cc, const int32_t *cmax, unsigned long long *rootkey) {
+  GS(v, nr) {
+    const int32_t c = cc[v];
+    const int64_t mid = ((int64_t)c + cmax[c]) / 2, d = (int64_t)v >= mid ? (int64_t)v - mid : mid - (int64_t)v;
+    atomicMin(&rootkey[c], ((unsigned long long)d << 32) | (uint32_t)v);
+  }
+}
+
 // ------------------------------------------------------------------ spanning forest (one CTA)
-// BFS from every component root (cc[v] == v), then subtree sizes (bottom-up), preorder numbers
+// BFS from every component's root (k_comp_root), then subtree sizes (bottom-up), preorder numbers
 // (top-down: children of u get consecutive ranges after pre(u)), and low/high = min/max preorder
 // number reachable from the subtree through one non-tree edge (bottom-up).  Levels are separated by
 // __syncthreads(), which also orders the global-memory atomics of the single block.
 __global__ void __launch_bounds__(TB, 1)
-    k_tree(int32_t nr, const int32_t *rp, const int32_t *col, const int32_t *cc, int32_t *parent, int32_t *order,
-           int32_t *lvl, int32_t *size, int32_t *pre, int32_t *low, int32_t *high, int32_t *out_levels) {
+    k_tree(int32_t nr, const int32_t *rp, const int32_t *col, const int32_t *cc, const unsigned long long *rootkey,
+           int32_t *parent, int32_t *order, int32_t *lvl, int32_t *size, int32_t *pre, int32_t *low, int32_t *high,
+           int32_t *out_levels) {
   using BS = cub::BlockScan<int32_t, TB>;
   __shared__ typename BS::TempStorage ts;
   __shared__ int32_t s_tail, s_carry;
   const int t = threadIdx.x;
   for (int32_t v = t; v < nr; v += TB) {
-    parent[v] = cc[v] == v ? -1 : -2;
+    parent[v] = (int32_t)(uint32_t)rootkey[cc[v]] == v ? -1 : -2;
     size[v] = 1;
   }
   if (t == 0) s_carry = 0;
   __syncthreads();
   for (int32_t b0 = 0; b0 < nr; b0 += TB) {   // roots, ascending
     const int32_t v = b0 + t;
-    const int32_t f = (v < nr && cc[v] == v) ? 1 : 0;
+    const int32_t f = (v < nr && (int32_t)(uint32_t)rootkey[cc[v]] == v) ? 1 : 0;
     int32_t off, tot;
     BS(ts).ExclusiveSum(f, off, tot);
     if (f) order[s_carry + off] = v;
@@ -592,7 +607,12 @@ ear_status_t bcc_prepare(ear_plan_s *p, int32_t P, cudaStream_t st) {
   EAR_LAUNCH(k_edges_all, grid_for(nr), NT, 0, st)(rp, col, nr, e, ne);
   EAR_TRY(cc_run(nr, e, ne, emax, cc, changed, st));
   // 2. spanning forest, preorder, low/high
-  EAR_LAUNCH(k_tree, 1, TB, 0, st)(nr, rp, col, cc, parent, order, lvl, size, pre, low, high, levels);
+  // rkey and size are scratch here (both are initialised again below / inside k_tree)
+  EAR_CUDA_TRY(dev_memset(size, 0, 4 * (size_t)nr, st));
+  EAR_CUDA_TRY(dev_memset(rkey, 0xFF, 8 * (size_t)nr, st));
+  EAR_LAUNCH(k_comp_maxid, grid_for(nr), NT, 0, st)(nr, cc, size);
+  EAR_LAUNCH(k_comp_root, grid_for(nr), NT, 0, st)(nr, cc, size, rkey);
+  EAR_LAUNCH(k_tree, 1, TB, 0, st)(nr, rp, col, cc, rkey, parent, order, lvl, size, pre, low, high, levels);
   // 3. auxiliary graph -> blocks
   EAR_CUDA_TRY(dev_memset(ne, 0, 4, st));
   EAR_LAUNCH(k_edges_aux, grid_for(nr), NT, 0, st)(rp, col, nr, parent, pre, size, low, high, e, ne);
