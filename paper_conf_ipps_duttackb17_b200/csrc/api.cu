@@ -3,6 +3,8 @@
 #include <cstring>
 #include <vector>
 
+#include <cstdlib>
+
 #include "common.cuh"
 
 namespace ear {
@@ -82,9 +84,28 @@ void ear_row_block(int32_t rows, int32_t nranks, int32_t rank, int32_t *begin, i
   if (end) *end = (int32_t)((int64_t)rows * (rank + 1) / nranks);
 }
 
+// The library's scratch (D, piece pool, expansion buffers) comes from the device's default stream-ordered
+// pool.  With its default release threshold (0) the pool hands its memory back to the driver at every
+// synchronisation and the next call maps it again; keep it instead (EAR_POOL_KEEP=0 restores the default).
+static void keep_pool_memory() {
+  static bool done[64] = {};
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64 || done[dev]) return;
+  done[dev] = true;
+  const char *e = getenv("EAR_POOL_KEEP");
+  if (e && atoi(e) == 0) return;
+  cudaMemPool_t pool;
+  if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
+    uint64_t keep = UINT64_MAX;
+    cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &keep);
+  }
+  cudaGetLastError();
+}
+
 ear_status_t ear_decompose(int32_t n, int64_t m, const int32_t *d_src, const int32_t *d_dst, const int32_t *d_w,
                            uint32_t flags, void *stream, ear_plan_t *out) {
   g_err[0] = 0;
+  keep_pool_memory();
   if (!out) { set_error("ear_decompose: out is NULL"); return EAR_EINVAL; }
   *out = nullptr;
   if (n < 1 || m < 0 || (m > 0 && (!d_src || !d_dst || !d_w)) || 2 * m > (int64_t)INT32_MAX) {

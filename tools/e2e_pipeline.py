@@ -11,6 +11,9 @@ hs, hd, hw = (torch.as_tensor(x).pin_memory() for x in (g.src, g.dst, g.w))
 hout = torch.empty((g.n, g.n), dtype=torch.int32, pin_memory=True)
 st = torch.cuda.current_stream()
 ea.apsp_full_host(g.n, hs, hd, hw, out=hout, flags=ea.FLAG_BCC, stream=st)
+if "--warm2" in sys.argv:   # two jobs in flight once: the memory pool reaches its pipelined size
+    for j in [ea.apsp_full_host_async(g.n, hs, hd, hw, out=hout, flags=ea.FLAG_BCC, stream=st) for _ in range(2)]:
+        j.wait()
 t0 = time.perf_counter()
 for _ in range(2):
     ea.apsp_full_host(g.n, hs, hd, hw, out=hout, flags=ea.FLAG_BCC, stream=st)
