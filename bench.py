@@ -380,7 +380,7 @@ def run_ours(args, rank, world, local_rank):
         nbuf = args.e2e_bufs or (2 if pipelined and psutil.virtual_memory().available > 2.5 * out_bytes else 1)
         houts = [torch.empty((rows, g.n), dtype=torch.int32, pin_memory=True) for _ in range(nbuf)]
         if pipelined:   # warm-up in the timed mode: two jobs in flight grow the library's memory pool to its
-            # steady-state size (fresh pool pages are scrubbed on the copy engines, behind the row copies)
+            # steady-state size (fresh pool pages appear to queue behind the row copies on the copy engines)
             wj = [ea.apsp_full_host_async(g.n, hs, hd, hw, out=houts[i % nbuf], row_begin=r0, row_end=r1,
                                           flags=flags, comm=comm, stream=stream) for i in range(2)]
             for j in wj:
