@@ -91,7 +91,10 @@ typedef struct {
  * two chain ends (left/right), its along-chain distance to each (reading C7) and its chain
  * (ear) id.  Terminal ids (tid) are assigned in increasing caller-id order.
  * Synchronises `stream` (N_r is data dependent).  On success *out is a new plan (caller destroys it
- * with ear_plan_destroy).  Errors: EAR_EINVAL (n < 1, m < 0, ids out of range, weight < 1),
+ * with ear_plan_destroy).  The library's device scratch comes from the device's default stream-ordered
+ * pool (cudaMallocAsync); the first call on a device sets that pool's release threshold to "keep"
+ * (EAR_POOL_KEEP=0 in the environment leaves it at the driver default), so freed scratch stays
+ * reserved for the next call instead of being mapped again.  Errors: EAR_EINVAL (n < 1, m < 0, ids out of range, weight < 1),
  * EAR_EOVERFLOW ((n-1)*max weight >= EAR_INF), EAR_ENOMEM, EAR_ECUDA. */
 ear_status_t ear_decompose(int32_t n, int64_t m, const int32_t *d_src, const int32_t *d_dst,
                            const int32_t *d_w, uint32_t flags, void *stream, ear_plan_t *out);
