@@ -42,7 +42,7 @@ typedef enum {
   EAR_EINVAL = -1,         /* bad argument: n < 1, m < 0, id out of [0,n), weight < 1, bad range */
   EAR_ENOMEM = -2,         /* device or host allocation failed */
   EAR_ECUDA = -3,          /* CUDA runtime / kernel error */
-  EAR_ENCCL = -4,          /* NCCL error */
+  EAR_ENCCL = -4,          /* communicator error (the caller's all-gather callback failed) */
   EAR_EOVERFLOW = -5,      /* (n-1) * max weight >= EAR_INF: distances might not fit */
   EAR_EUNSUPPORTED = -6    /* unsupported configuration (e.g. misaligned pointer where required) */
 } ear_status_t;
@@ -65,7 +65,7 @@ enum {
 };
 
 typedef struct ear_plan_s *ear_plan_t; /* Reduce(G) result: descriptors + reduced edge list (device) */
-typedef struct ear_comm_s *ear_comm_t; /* NCCL communicator for row-block sharding; NULL = 1 GPU */
+typedef struct ear_comm_s *ear_comm_t; /* peer-memory communicator for row-block sharding; NULL = 1 GPU */
 
 /* Summary of a plan.  n_reduced_padded depends on the number of ranks (padding to EAR_TILE*nranks). */
 typedef struct {
@@ -249,11 +249,26 @@ ear_status_t ear_job_wait(ear_job_t job);
  * Contiguous near-equal split of `rows` rows over nranks: rank gets [*begin, *end). */
 void ear_row_block(int32_t rows, int32_t nranks, int32_t rank, int32_t *begin, int32_t *end);
 
-/* NCCL unique id (128 bytes) created on rank 0 and distributed by the caller (torch.distributed). */
-ear_status_t ear_comm_unique_id(uint8_t id[128]);
-/* Create this rank's communicator on the current CUDA device.  Collective over all ranks. */
-ear_status_t ear_comm_init(const uint8_t id[128], int32_t nranks, int32_t rank, ear_comm_t *out);
+/* Host all-gather supplied by the caller (the Python binding uses torch.distributed): every rank passes
+ * `bytes` bytes at `send`; on return `recv` holds rank r's bytes at recv + r * bytes.  Collective over
+ * all ranks; returns 0 on success.  The library calls it only inside collective calls (ear_comm_init,
+ * and apsp_reduced / apsp_full / ear_gather_reduced when a larger exchange window is needed) to trade
+ * CUDA IPC handles -- never on the data path. */
+typedef int32_t (*ear_allgather_fn)(const void *send, void *recv, int64_t bytes, void *ctx);
+
+/* Create this rank's communicator on the current CUDA device: the peer-memory transport of the
+ * row-block-sharded FW.  Every rank owns a device window exported by CUDA IPC and
+ * mapped by every other rank (NVLink/NVSwitch peer memory between GPUs; several ranks may share one
+ * GPU); each FW round a rank stores its phase-2-updated pieces of the pivot row block straight into
+ * every peer's window and raises a flag (the per-round broadcast of the pieces), and the final D is
+ * all-gathered by reading the peers' owned tile rows.  Collective over all ranks; nranks <= EAR_MAX_RANKS;
+ * `allgather` (with `ctx`) may be NULL only for nranks == 1 and must stay valid until
+ * ear_comm_destroy.  Errors: EAR_EINVAL, EAR_ENCCL (the callback failed), EAR_ECUDA. */
+#define EAR_MAX_RANKS 16
+ear_status_t ear_comm_init(int32_t nranks, int32_t rank, ear_allgather_fn allgather, void *ctx, ear_comm_t *out);
 ear_status_t ear_comm_info(ear_comm_t comm, int32_t *nranks, int32_t *rank);
+/* Synchronises the device, unmaps the peers' windows and frees this rank's (no other rank may still be
+ * using the communicator in a call). */
 void ear_comm_destroy(ear_comm_t comm);
 
 /* ---------------------------------------------------------------- profiling (bench.py, tests)

@@ -14,6 +14,10 @@ Functions (paper = /root/reference/PAPER.md, ``P:NN`` = line NN):
 * :func:`apsp` -- all rows.
 * :func:`reduce_graph` -- ``G^r = Reduce(G)`` by a sequential chain walk as defined
   (readings C3-C7 in DESIGN.md).
+* :func:`certify_rows` -- a CHECKER: how many entries of candidate rows violate the Bellman optimality
+  equations of S on the original graph (P:41, P:109 restated as a fixed point; SURVEY 8.c pin P4).
+  Its only solution with integer weights >= 1 is S itself, and it costs O(N + M) per row, so it
+  certifies whole N x N matrices (cfg4, cfg5) where Dijkstra from every source would take minutes.
 
 Pinned by ``tests/test_oracle_pins.py``: brute-force Floyd-Warshall and exhaustive enumeration of
 all small graphs (P1), closed forms (P2), invariants (P3), the Bellman certificate (P4), scipy's
@@ -57,6 +61,9 @@ def _load():
         lib.oracle_num_threads.restype = ctypes.c_int
         lib.oracle_reduce.argtypes = [ctypes.c_int32, ctypes.c_int64, P, P, P] + [P] * 10 + [ctypes.c_int64, P]
         lib.oracle_reduce.restype = ctypes.c_int
+        lib.oracle_certify_rows.argtypes = [ctypes.c_int32, ctypes.c_int64, P, P, P, ctypes.c_int32, P, P,
+                                            ctypes.c_int64, ctypes.c_int32, P, P]
+        lib.oracle_certify_rows.restype = ctypes.c_int64
         _lib = lib
     return _lib
 
@@ -92,6 +99,26 @@ def apsp_rows(n: int, src, dst, w, rows, nthreads: int = 0) -> np.ndarray:
 def apsp(n: int, src, dst, w, nthreads: int = 0) -> np.ndarray:
     """The full ``S`` (n x n int32)."""
     return apsp_rows(n, src, dst, w, np.arange(n, dtype=np.int32), nthreads)
+
+
+def certify_rows(n: int, src, dst, w, rows, D: np.ndarray, nthreads: int = 0, per_row: bool = False):
+    """Check candidate rows ``D[i] == S[rows[i], :]`` through the Bellman optimality equations (see the
+    module docstring).  ``D``: int32, shape (len(rows), >= n), C-contiguous rows.  Returns
+    ``(violations, (i, t) of the first one or None)`` -- plus the per-row violation counts with
+    ``per_row``."""
+    src, dst, w = _edges(src, dst, w)
+    rows = np.ascontiguousarray(rows, dtype=np.int32)
+    if D.dtype != np.int32 or D.ndim != 2 or D.shape[0] < len(rows) or D.shape[1] < n or D.strides[1] != 4:
+        raise ValueError("D must be an int32 (rows, >= n) array with unit column stride")
+    first = np.full(2, -1, dtype=np.int64)
+    rb = np.zeros(len(rows), dtype=np.int64) if per_row else None
+    bad = _load().oracle_certify_rows(n, len(src), _ptr(src), _ptr(dst), _ptr(w), len(rows), _ptr(rows),
+                                      D.ctypes.data_as(ctypes.c_void_p), D.strides[0] // 4, nthreads, _ptr(first),
+                                      _ptr(rb) if per_row else None)
+    if bad < 0:
+        raise ValueError(f"oracle_certify_rows failed with status {bad}")
+    res = (int(bad), (None if first[0] < 0 else (int(first[0]), int(first[1]))))
+    return res + (rb,) if per_row else res
 
 
 @dataclass

@@ -31,6 +31,19 @@
  *                     Pins: Fig. 4 chains, the cyclomatic identity of Lemma 3.1's proof
  *                      and brute-force checks in tests/test_oracle_pins.py.
  *
+ *  oracle_certify_rows  a CHECKER, not a solver: whether candidate rows of S satisfy the Bellman
+ *                     optimality equations of shortest paths in the ORIGINAL graph -- the definition
+ *                     of S restated as a fixed point (SURVEY 8.c pin P4):
+ *                       D[s][s] = 0;  D[s][t] = min over arcs (u,t) of D[s][u] + w(u,t)  (t != s),
+ *                       ORACLE_INF when no u has a finite D[s][u].
+ *                     With integer weights >= 1 the true distances are its ONLY solution: an entry
+ *                     satisfying it is at most the weight of any s-t path (induction along the path),
+ *                     and a finite entry is the weight of the walk spelled out by its strictly
+ *                     decreasing chain of tight predecessors, which can only end at s.  O(N + M) per
+ *                     row instead of Dijkstra's O(M log N): it certifies whole N x N matrices (cfg4,
+ *                     cfg5) in seconds.  Pins: tests/test_oracle_pins.py (accepts the oracle's rows,
+ *                     rejects every single-entry perturbation, exhaustive small graphs).
+ *
  * Build: gcc -O2 -fopenmp -shared -fPIC -o oracle/liboracle.so oracle/apsp_oracle.c
  */
 #include <stdint.h>
@@ -328,4 +341,62 @@ done:
   counts[0] = nterm; counts[1] = nre; counts[2] = nchains; counts[3] = promoted;
   free(path); free(pre); free(s_start); free(s_nb);
   return status;
+}
+
+/* ------------------------------------------------------------------ Bellman certificate (checker)
+ * Rows i < nrows of D (leading dimension ldd) are candidate rows S[rows[i], :].  Returns the number of
+ * entries that violate the equations in the header (0: every row is exactly S), or a negative status;
+ * first[0..1] = (i, t) of the first violation found (by row index); row_bad (may be NULL) gets the
+ * violations of every row.  */
+int64_t oracle_certify_rows(int32_t n, int64_t m, const int32_t *src, const int32_t *dst, const int32_t *w,
+                            int32_t nrows, const int32_t *rows, const int32_t *D, int64_t ldd, int32_t nthreads,
+                            int64_t *first, int64_t *row_bad_out) {
+  if (validate(n, m, src, dst, w)) return -1;
+  for (int32_t r = 0; r < nrows; ++r)
+    if (rows[r] < 0 || rows[r] >= n) return -1;
+  if (ldd < n) return -1;
+  adj_t g;
+  if (adj_build(&g, n, m, src, dst, w)) { adj_free(&g); return -2; }
+#ifdef _OPENMP
+  if (nthreads > 0) omp_set_num_threads(nthreads);
+#endif
+  int64_t bad = 0;
+  first[0] = -1;
+  first[1] = -1;
+#pragma omp parallel for schedule(dynamic, 4) reduction(+ : bad)
+  for (int32_t i = 0; i < nrows; ++i) {
+    const int32_t s = rows[i];
+    const int32_t *d = D + (int64_t)i * ldd;
+    int64_t row_bad = 0;
+    int32_t first_t = -1;
+    for (int32_t t = 0; t < n; ++t) {
+      int64_t expect;
+      if (t == s) {
+        expect = 0;
+      } else {
+        int64_t best = ORACLE_INF;   /* min over the arcs (u, t); the graph is undirected */
+        for (int64_t a = g.start[t]; a < g.start[t + 1]; ++a) {
+          const int32_t u = g.nbr[a];
+          const int64_t du = d[u];
+          if (u == t || du < 0 || du >= ORACLE_INF) continue;   /* self-loop, or no finite path to u */
+          if (du + g.wt[a] < best) best = du + g.wt[a];
+        }
+        expect = best;
+      }
+      if ((int64_t)d[t] != expect) {
+        if (first_t < 0) first_t = t;
+        ++row_bad;
+      }
+    }
+    if (row_bad_out) row_bad_out[i] = row_bad;
+    if (row_bad) {
+#pragma omp critical
+      {
+        if (first[0] < 0 || i < first[0]) { first[0] = i; first[1] = first_t; }
+      }
+      bad += row_bad;
+    }
+  }
+  adj_free(&g);
+  return bad;
 }

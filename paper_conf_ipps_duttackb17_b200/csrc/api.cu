@@ -4,6 +4,7 @@
 #include <vector>
 
 #include <cstdlib>
+#include <mutex>
 
 #include "common.cuh"
 
@@ -39,21 +40,6 @@ int32_t padded(const ear_plan_s *p, int32_t nranks) {
 
 bool aligned16(const void *p) { return ((uintptr_t)p & 15u) == 0; }
 
-// Scratch (D, sort buffers, pivot rows) comes from the device's default stream-ordered pool.  Keep
-// freed blocks cached instead of returning them to the driver at every synchronisation (the
-// default release threshold 0 would re-map the 3.6 GB D of cfg4 on every call).
-void ensure_pool() {
-  static bool done[64] = {false};
-  int dev = 0;
-  if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64 || done[dev]) return;
-  cudaMemPool_t pool;
-  if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
-    uint64_t thr = UINT64_MAX;
-    cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
-  }
-  done[dev] = true;
-}
-
 }  // namespace
 }  // namespace ear
 
@@ -84,23 +70,31 @@ void ear_row_block(int32_t rows, int32_t nranks, int32_t rank, int32_t *begin, i
   if (end) *end = (int32_t)((int64_t)rows * (rank + 1) / nranks);
 }
 
+}  // extern "C"
+
+namespace {
 // The library's scratch (D, piece pool, expansion buffers) comes from the device's default stream-ordered
 // pool.  With its default release threshold (0) the pool hands its memory back to the driver at every
-// synchronisation and the next call maps it again; keep it instead (EAR_POOL_KEEP=0 restores the default).
-static void keep_pool_memory() {
-  static bool done[64] = {};
+// synchronisation and the next call maps it again; keep it instead (EAR_POOL_KEEP=0 keeps the driver
+// default).  Once per device, thread-safe.
+void keep_pool_memory() {
+  static std::once_flag once[64];
   int dev = 0;
-  if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64 || done[dev]) return;
-  done[dev] = true;
-  const char *e = getenv("EAR_POOL_KEEP");
-  if (e && atoi(e) == 0) return;
-  cudaMemPool_t pool;
-  if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
-    uint64_t keep = UINT64_MAX;
-    cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &keep);
-  }
-  cudaGetLastError();
+  if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return;
+  std::call_once(once[dev], [dev] {
+    const char *e = getenv("EAR_POOL_KEEP");
+    if (e && atoi(e) == 0) return;
+    cudaMemPool_t pool;
+    if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
+      uint64_t keep = UINT64_MAX;
+      cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &keep);
+    }
+    cudaGetLastError();
+  });
 }
+}  // namespace
+
+extern "C" {
 
 ear_status_t ear_decompose(int32_t n, int64_t m, const int32_t *d_src, const int32_t *d_dst, const int32_t *d_w,
                            uint32_t flags, void *stream, ear_plan_t *out) {
@@ -116,7 +110,6 @@ ear_status_t ear_decompose(int32_t n, int64_t m, const int32_t *d_src, const int
     set_error("ear_decompose: EAR_FLAG_SSSP and EAR_FLAG_BCC are exclusive");
     return EAR_EINVAL;
   }
-  ensure_pool();
   ear_plan_s *p = new ear_plan_s;
   cudaGetDevice(&p->device);
   int sp = prof_begin(PK_DECOMPOSE, (cudaStream_t)stream);
@@ -240,7 +233,7 @@ ear_status_t apsp_reduced_rank_timing(ear_plan_t p, int32_t nranks, int32_t rank
     set_error("apsp_reduced_rank_timing: bad argument");
     return EAR_EINVAL;
   }
-  return fw_rank_timing(p, padded(p, nranks), nranks, rank, (cudaStream_t)stream);
+  return fw_rank_timing(p, padded(p, nranks), nranks, rank, (p->flags & EAR_FLAG_FW32) != 0, (cudaStream_t)stream);
 }
 
 int32_t ear_owned_tile_rows(int32_t n_reduced_padded, int32_t nranks, int32_t rank) {
@@ -302,12 +295,11 @@ static ear_status_t solve_rows(ear_plan_s *p, int32_t row_begin, int32_t row_end
     EAR_CUDA_TRY(cudaMallocAsync((void **)&Dfull, sizeof(int32_t) * (size_t)Np * Np, st));
     s = bcc_solve(p, comm, Dfull, Np, Np, 0, Np, nullptr, st);
   } else {
-    const int32_t nown = shard_nown(Np / TILE, P, comm->rank);
+    // the owned rows live in this rank's exchange window, where the gather reads them
     EAR_CUDA_TRY(cudaMallocAsync((void **)&Dfull, sizeof(int32_t) * (size_t)Np * Np, st));
-    EAR_CUDA_TRY(cudaMallocAsync((void **)&D, sizeof(int32_t) * (size_t)std::max(nown, 1) * TILE * Np, st));
-    s = apsp_reduced(p, D, Np, comm, st);
+    s = fw_shard_buffer(comm, Np, st, &D);
+    if (s == EAR_OK) s = apsp_reduced(p, D, Np, comm, st);
     if (s == EAR_OK) s = ear_gather_reduced(p, D, Np, Dfull, Np, comm, st);
-    cudaFreeAsync(D, st);
   }
   if (s == EAR_OK && d_out) s = expand_ears(p, Dfull, Np, row_begin, row_end, d_out, ldo, st);
   if (D_keep && s == EAR_OK) {
@@ -353,8 +345,10 @@ namespace {
 // the device's host-copy stream: every job's D2H copies, in issue order
 cudaStream_t host_copy_stream() {
   static cudaStream_t cs[64] = {};
+  static std::mutex mu;
   int dev = 0;
   if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return nullptr;
+  std::lock_guard<std::mutex> lk(mu);
   if (!cs[dev] && cudaStreamCreateWithFlags(&cs[dev], cudaStreamNonBlocking) != cudaSuccess) cs[dev] = nullptr;
   return cs[dev];
 }

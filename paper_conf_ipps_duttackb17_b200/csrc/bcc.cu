@@ -704,10 +704,6 @@ ear_status_t bcc_prepare(ear_plan_s *p, int32_t P, cudaStream_t st) {
   return EAR_OK;
 }
 
-ear_status_t fw_sharded_gather(const int32_t *S, int64_t ldd, int32_t Np, int32_t *Df, int64_t ldf, ear_comm_s *comm,
-                               cudaStream_t st);
-std::vector<int32_t> shard_rows(int32_t nt, int32_t P, int32_t rank);
-int32_t shard_nown(int32_t nt, int32_t P, int32_t rank);
 
 // The paper's order inside a big piece (G is split into its biconnected components and EACH is
 // then reduced): a vertex of degree >= 3 in G^r can have degree 2 inside its block (an articulation
@@ -762,17 +758,12 @@ static ear_status_t reduce_solve(const ear_plan_s *p, int32_t n, int64_t m, cons
       if (s == EAR_OK) s = fw_single(D, Np, Np, st, nullptr, q->n_reduced, allow16, q);   // connected
     } else {
       const std::vector<int32_t> own = shard_rows(Np / TILE, P, comm->rank);
-      int32_t *S = nullptr;
-      if (cudaMallocAsync((void **)&S, sizeof(int32_t) * std::max<size_t>(own.size(), 1) * TILE * Np, st) !=
-          cudaSuccess) {
-        set_error("bcc_solve: out of device memory (re-reduced piece)");
-        s = EAR_ENOMEM;
-      }
+      int32_t *S = nullptr;   // the owned rows live in this rank's exchange window (read there by the gather)
+      s = fw_shard_buffer(comm, Np, st, &S);
       for (size_t j = 0; j < own.size() && s == EAR_OK; ++j)
         s = fw_init_D(q, S + (int64_t)j * TILE * Np, Np, Np, own[j] * TILE, TILE, st);
       if (s == EAR_OK) s = fw_sharded_auto(S, Np, Np, comm, nullptr, q->n_reduced, allow16, st, q);
       if (s == EAR_OK) s = fw_sharded_gather(S, Np, Np, D, Np, comm, st);
-      if (S) cudaFreeAsync(S, st);
     }
   }
   if (s == EAR_OK) s = expand(q, D, Np, 0, n, M, ld, st, PK_REREDUCE);
@@ -827,6 +818,7 @@ ear_status_t bcc_solve(ear_plan_s *p, ear_comm_s *comm, int32_t *D, int64_t ldd,
   EAR_TRY(sprep);
   ear_bcc_s *b = p->bcc;
   const int32_t nr = p->n_reduced;
+  EAR_CUDA_TRY(smem_attr((const void *)k_piece_fw, SMALL * SMALL * 4));
   int32_t *pool = nullptr;
   EAR_CUDA_TRY(cudaMallocAsync((void **)&pool, sizeof(int32_t) * (size_t)std::max<int64_t>(b->pool_ints, 4), st));
   ear_status_t s = EAR_OK;
@@ -834,11 +826,6 @@ ear_status_t bcc_solve(ear_plan_s *p, ear_comm_s *comm, int32_t *D, int64_t ldd,
   EAR_LAUNCH(k_fill_pool, grid_for(b->pool_ints / 4 + 1), NT, 0, st)(pool, b->pool_ints);
   EAR_LAUNCH(k_pool_init, grid_for(std::max(nr, b->n_arcs)), NT, 0, st)(nr, b->cinfo, b->ridx, b->hp, b->pld,
                                                                          b->pbase, b->arcs, b->n_arcs, pool);
-  static bool attr = false;
-  if (!attr) {
-    cudaFuncSetAttribute(k_piece_fw, cudaFuncAttributeMaxDynamicSharedMemorySize, SMALL * SMALL * 4);
-    attr = true;
-  }
   if (b->n_pieces > 0)
     EAR_LAUNCH(k_piece_fw, b->n_pieces, NT, SMALL * SMALL * 4, st)(b->n_pieces, b->psize, b->pld, b->pbase, pool);
   prof_end(sp, st, 0);
@@ -857,13 +844,8 @@ ear_status_t bcc_solve(ear_plan_s *p, ear_comm_s *comm, int32_t *D, int64_t ldd,
     if (comm && i == 0) {   // the largest piece: sharded over the ranks, then gathered everywhere
       const int32_t nt = ld / TILE;
       std::vector<int32_t> own = shard_rows(nt, P, comm->rank);
-      int32_t *S = nullptr;
-      if (cudaMallocAsync((void **)&S, sizeof(int32_t) * (size_t)std::max<size_t>(own.size(), 1) * TILE * ld, st) !=
-          cudaSuccess) {
-        set_error("bcc_solve: out of device memory");
-        s = EAR_ENOMEM;
-        break;
-      }
+      int32_t *S = nullptr;   // the owned rows live in this rank's exchange window (read there by the gather)
+      s = fw_shard_buffer(comm, ld, st, &S);
       for (size_t j = 0; j < own.size() && s == EAR_OK; ++j)
         if (cudaMemcpyAsync(S + (int64_t)j * TILE * ld, M + (int64_t)own[j] * TILE * ld,
                             sizeof(int32_t) * (size_t)TILE * ld, cudaMemcpyDeviceToDevice, st) != cudaSuccess)
@@ -871,7 +853,6 @@ ear_status_t bcc_solve(ear_plan_s *p, ear_comm_s *comm, int32_t *D, int64_t ldd,
       if (s == EAR_OK)   // a piece is connected: no labels
         s = fw_sharded_auto(S, ld, ld, comm, nullptr, b->h_psize[id], !(p->flags & EAR_FLAG_FW32), st);
       if (s == EAR_OK) s = fw_sharded_gather(S, ld, ld, M, ld, comm, st);
-      cudaFreeAsync(S, st);
     } else {
       s = fw_single(M, ld, ld, st, nullptr, b->h_psize[id], !(p->flags & EAR_FLAG_FW32));   // a piece is connected
     }

@@ -39,6 +39,12 @@ struct __align__(16) VDesc {
   int32_t p, cp, q, cq;
 };
 
+// up to EAR_MAX_RANKS pointers, passed to kernels by value (one per rank: peer windows, destinations)
+struct PeerPtrs {
+  char *p[EAR_MAX_RANKS];
+  int32_t n;
+};
+
 }  // namespace ear
 
 struct ear_bcc_s;   // bcc.cu: block structure of G^r and the piece layout (EAR_FLAG_BCC)
@@ -78,12 +84,18 @@ struct ear_plan_s {
   int32_t cc_np = 0;
 };
 
+// Library-owned communicator (comm.cu): the ranks' peer-mapped windows and the flag sequences.
 struct ear_comm_s {
-  void *nccl = nullptr;  // ncclComm_t
   int32_t nranks = 1;
   int32_t rank = 0;
   int device = 0;
-  cudaStream_t comm_stream = nullptr;
+  ear_allgather_fn allgather = nullptr;   // caller's host all-gather (handle exchange only)
+  void *ctx = nullptr;
+  char *win = nullptr;                    // this rank's window (cudaMalloc, IPC-exported)
+  size_t win_bytes = 0;
+  char *peer[EAR_MAX_RANKS] = {};         // every rank's window mapped here (peer[rank] == win)
+  int32_t np = 0;                         // Np the window layout is cut for (comm_reserve)
+  uint64_t seq_pieces = 0, seq_tile = 0, seq_barrier = 0, seq_check = 0;   // flag values, same on every rank
 };
 
 namespace ear {
@@ -135,14 +147,17 @@ ear_status_t fw_single(int32_t *D, int64_t ldd, int32_t Np, cudaStream_t stream,
                        int32_t n_real = 0, bool allow16 = false, ear_plan_s *plan = nullptr);
 ear_status_t reduced_labels(ear_plan_s *p, int32_t Np, cudaStream_t st, const int32_t **out);
 // row-block sharding: rank r owns the tile rows ti with (ti mod 2P) in {r, 2P-1-r} (zig-zag), stored
-// ascending as 128-row blocks
-ear_status_t fw_sharded(int32_t *S, int64_t ldd, int32_t Np, ear_comm_s *comm, cudaStream_t stream);
-// the 16-bit sharded schedule first (allow16; lab / n_real as for fw_single), else fw_sharded
+// ascending as 128-row blocks; the exchange runs over the communicator's peer windows (comm.cu)
+std::vector<int32_t> shard_rows(int32_t nt, int32_t P, int32_t rank);
+// the packed schedule first (allow16; lab / n_real as for fw_single), else the int32 one; collective
 ear_status_t fw_sharded_auto(int32_t *S, int64_t ldd, int32_t Np, ear_comm_s *comm, const int32_t *lab,
                              int32_t n_real, bool allow16, cudaStream_t stream, ear_plan_s *plan = nullptr);
+// every rank's owned upper tiles -> the full matrix Df on every rank (peer reads + mirror); collective
 ear_status_t fw_sharded_gather(const int32_t *S, int64_t ldd, int32_t Np, int32_t *Df, int64_t ldf, ear_comm_s *comm,
                                cudaStream_t stream);
-ear_status_t fw_rank_timing(const ear_plan_s *plan, int32_t Np, int32_t P, int32_t rank, cudaStream_t stream);
+// this rank's owned-row storage inside its window (no copy at the gather); collective
+ear_status_t fw_shard_buffer(ear_comm_s *comm, int32_t Np, cudaStream_t stream, int32_t **S);
+ear_status_t fw_rank_timing(const ear_plan_s *plan, int32_t Np, int32_t P, int32_t rank, bool fw32, cudaStream_t stream);
 ear_status_t fw_sharded_emulated(ear_plan_s *plan, int32_t *D, int64_t ldd, int32_t Np, int32_t P,
                                  cudaStream_t stream);
 int32_t shard_nown(int32_t nt, int32_t P, int32_t rank);
@@ -163,9 +178,20 @@ ear_status_t expand(const ear_plan_s *plan, const int32_t *D, int64_t ldd, int32
                     int32_t row_end, int32_t *out, int64_t ldo, cudaStream_t stream, int prof_kind = PK_EXPAND);
 ear_status_t query_pairs(const ear_plan_s *plan, const int32_t *D, int64_t ldd, int64_t npairs, const int32_t *qs,
                          const int32_t *qt, int32_t *out, cudaStream_t stream);
-// comm.cu
-ear_status_t comm_bcast(ear_comm_s *comm, int32_t *buf, int64_t count, int32_t root, cudaStream_t stream);
-ear_status_t comm_allgather(ear_comm_s *comm, const int32_t *send, int32_t *recv, int64_t count,
-                            cudaStream_t stream);
-ear_status_t comm_allreduce_min(ear_comm_s *comm, int32_t *buf, int64_t count, cudaStream_t stream);
+// comm.cu -- peer-memory transport (window layout in comm.cu)
+enum { SLOT_PIECES = 0, SLOT_TILE = 64, SLOT_BARRIER = 128, SLOT_CHECK = 192 };
+size_t comm_win_bytes(int32_t Np, int32_t nown);
+ear_status_t comm_reserve(ear_comm_s *c, int32_t Np, int32_t nown, cudaStream_t st);   // collective
+char *comm_L(ear_comm_s *c, int p, int b);          // rank p's L[b] as mapped here
+char *comm_stage(ear_comm_s *c, int p, int b);      // rank p's stage[b]
+int32_t *comm_region(ear_comm_s *c, int p);         // rank p's owned-rows region
+PeerPtrs comm_flags_all(ear_comm_s *c);             // every rank's window base (flag slots at offset 0)
+ear_status_t comm_signal(ear_comm_s *c, int32_t slot, uint64_t value, cudaStream_t st);
+ear_status_t comm_wait(ear_comm_s *c, int32_t slot, uint64_t value, cudaStream_t st);
+ear_status_t comm_wait_one(ear_comm_s *c, int32_t slot, uint64_t value, cudaStream_t st);
+ear_status_t comm_barrier(ear_comm_s *c, cudaStream_t st);
+// helpers (prof.cu): per-device SM count; cudaFuncSetAttribute(max dynamic smem) once
+// per (device, kernel), thread-safe
+int num_sms();
+cudaError_t smem_attr(const void *kernel, int bytes);
 }  // namespace ear

@@ -73,7 +73,6 @@ __device__ __forceinline__ int32_t *row_ptr(int32_t *base, int32_t r, uint32_t l
 // items instead of a partial wave of whole row groups.
 struct ExpandWork {
   int32_t *counter;
-  int32_t segmajor;   // > 0: every row group in segmajor column segments, items segment-major
   int32_t n_full, n_items, nseg, seg_w;
 };
 
@@ -99,12 +98,7 @@ __global__ void __launch_bounds__(NT, EXP_MINB) k_expand(const int32_t *__restri
   const int32_t item = item_sh;
   if (item >= W.n_items) break;
   int32_t rg = item, col_b = 0, col_e = n;
-  if (W.segmajor > 0) {
-    const int32_t groups = W.n_items / W.segmajor;
-    rg = item % groups;
-    col_b = (item / groups) * W.seg_w;
-    col_e = min(n, col_b + W.seg_w);
-  } else if (item >= W.n_full) {
+  if (item >= W.n_full) {
     rg = W.n_full + (item - W.n_full) / W.nseg;
     col_b = ((item - W.n_full) % W.nseg) * W.seg_w;
     col_e = min(n, col_b + W.seg_w);
@@ -281,31 +275,16 @@ __global__ void k_query_pairs(const int32_t *__restrict__ D, int64_t ldd, const 
 }
 
 
-bool g_attr_set = false;
-
-int env_int_ex(const char *name, int dflt) {
-  const char *e = getenv(name);
-  return e ? atoi(e) : dflt;
-}
-
 }  // namespace
 
 ear_status_t expand(const ear_plan_s *plan, const int32_t *D, int64_t ldd, int32_t row_begin, int32_t row_end,
                     int32_t *out, int64_t ldo, cudaStream_t st, int prof_kind) {
   const int32_t rows = row_end - row_begin;
   if (rows <= 0) return EAR_OK;
-  if (!g_attr_set) {
-    EAR_CUDA_TRY(cudaFuncSetAttribute(k_expand, cudaFuncAttributeMaxDynamicSharedMemorySize, EXP_SMEM));
-    g_attr_set = true;
-  }
-  static int slots = 0;   // resident CTAs per device (all B200s of a box alike)
-  if (!slots) {
-    int dev = 0, sms = 0, per = 0;
-    EAR_CUDA_TRY(cudaGetDevice(&dev));
-    EAR_CUDA_TRY(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
-    EAR_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_expand, NT, EXP_SMEM));
-    slots = std::max(1, sms * std::max(per, 1));
-  }
+  EAR_CUDA_TRY(smem_attr((const void *)k_expand, EXP_SMEM));
+  int per = 0;
+  EAR_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_expand, NT, EXP_SMEM));
+  const int32_t slots = std::max(1, num_sms() * std::max(per, 1));   // resident CTAs: one persistent wave
   const int32_t groups = (int32_t)ceil_div(rows, RB);
   ExpandWork W{};
   W.seg_w = (int32_t)round_up(ceil_div(plan->n, 8), CHUNK);
@@ -313,12 +292,6 @@ ear_status_t expand(const ear_plan_s *plan, const int32_t *D, int64_t ldd, int32
   const int32_t nsplit = std::min(groups, slots);
   W.n_full = groups - nsplit;
   W.n_items = W.n_full + nsplit * W.nseg;
-  static const int segs = env_int_ex("EAR_EXPAND_SEGS", 0);   // development knob: segment-major items
-  if (segs > 0) {
-    W.seg_w = (int32_t)round_up(ceil_div(plan->n, segs), CHUNK);
-    W.segmajor = (int32_t)ceil_div(plan->n, W.seg_w);
-    W.n_items = groups * W.segmajor;
-  }
   EAR_CUDA_TRY(cudaMallocAsync((void **)&W.counter, sizeof(int32_t), st));
   EAR_CUDA_TRY(dev_memset(W.counter, 0, sizeof(int32_t), st));
   const unsigned grid = (unsigned)std::min<int64_t>(W.n_items, slots);

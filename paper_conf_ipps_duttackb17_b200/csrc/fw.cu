@@ -1,27 +1,32 @@
 // Phase II -- S^r = APSP(G^r) (Alg. 1 lines 4-7) as a three-phase blocked min-plus
-// Floyd-Warshall (blocked FW of [23], cited at P:60) over 128 x 128 int32 tiles on sm_100a.
+// Floyd-Warshall (blocked FW of [23], cited at P:60) over 128 x 128 tiles on sm_100a.
 //
 //   D init   INF everywhere, 0 on the diagonal, atomicMin of the G^r arcs (keep the shortest of
 //            parallel edges).
 //   round k  phase 1  closure of the pivot tile (k,k): serial kk loop in one CTA; the matrix is
-//                     symmetric (undirected G), so row kk doubles as column kk and one smem row
-//                     buffer (double-buffered) broadcasts the pivot each step;
+//                     symmetric (undirected G), so row kk doubles as column kk;
 //            phase 2  pivot-row tiles (k,j): C = min(C, P (x) C) with the CLOSED pivot P -- a single
-//                     min-plus product, no serial dependency (closure argument in DESIGN.md);
+//                     min-plus product, no serial dependency (closure argument in DESIGN.md sec. 6);
 //            phase 3  remaining tiles (i,j): C = min(C, D[i,K] (x) D[K,j]).
-//   Both phase 2 and 3 run the same register-blocked min-plus tile kernel: 256 threads, 8x8 int32
-//   accumulators per thread, operands streamed through double-buffered shared memory by cp.async in
-//   32-deep k-chunks; one VIADDMNMX (c = min(c, a + b)) per min-plus.  Because D is symmetric,
-//   D[i,K] = D[K,i]^T: both operands are slices of the pivot ROW block, which is also the only
-//   block a multi-GPU round has to broadcast.  On one GPU only the upper triangle of tiles is
-//   computed and each result is written twice (tile and transposed mirror): half the min-plus work.
+//   Because D is symmetric, D[i,K] = D[K,i]^T: both operands of every tile update are slices of the
+//   pivot ROW block, which is also the only block a sharded round exchanges.  On one GPU only the upper
+//   triangle of tiles is computed and each result is written twice (tile and transposed mirror).
+//
+// One persistent, dynamically scheduled, TMA-fed tile kernel (k_fw_tiles) serves phases 2 and 3 in
+// two element types (fragment policies): Frag32 (int32, one VIADDMNMX per min-plus) and Frag16 (packed
+// u16x2 on a copy of D capped at C16 = 0x7FFF, two min-plus per VIADDMNMX.U16x2; exact below the cap,
+// DESIGN.md sec. 6d).  Both run the same lookahead schedule: round k+1's pivot chain on a per-call side
+// stream while round k's remaining tiles proceed.  Every piece of per-call state (side stream, events,
+// tile counters, precheck word) belongs to the call, so distinct calls on one device are independent.
 #include <cuda.h>
 #include <cudaTypedefs.h>
+#include <unistd.h>
 
 #include <algorithm>
+#include <cmath>
 #include <cstdio>
 #include <cstdlib>
-#include <cmath>
+#include <mutex>
 #include <vector>
 
 #include "common.cuh"
@@ -30,6 +35,7 @@ namespace ear {
 namespace {
 
 constexpr int NT = 256;
+constexpr uint32_t C16 = 0x7FFF;   // cap of the packed FW: a + b <= 0xFFFE never wraps for a, b <= C16
 
 __global__ void k_init_D(int32_t *D, int64_t ldd, int32_t Np, int32_t row0, int32_t rows) {
   int64_t total = (int64_t)rows * (Np / 4);
@@ -53,110 +59,8 @@ __global__ void k_init_edges(const int32_t *ru, const int32_t *rv, const int32_t
 
 __device__ __forceinline__ int32_t mp(int32_t a, int32_t b, int32_t c) { return __viaddmin_s32(a, b, c); }
 
-// ------------------------------------------------------------------------------ phase 1
-// Closure of the 128x128 pivot tile at T (leading dimension ldt), in place.
-__global__ void __launch_bounds__(NT, 1) k_fw_phase1(int32_t *T, int64_t ldt) {
-  __shared__ __align__(16) int32_t rowbuf[2][TILE];
-  const int tx = threadIdx.x & 15, ty = threadIdx.x >> 4;
-  int32_t c[8][8];
-#pragma unroll
-  for (int r = 0; r < 8; ++r) {
-    const int i = (r < 4 ? 0 : 64) + ty * 4 + (r & 3);
-    const int4 lo = *reinterpret_cast<const int4 *>(T + (int64_t)i * ldt + tx * 4);
-    const int4 hi = *reinterpret_cast<const int4 *>(T + (int64_t)i * ldt + 64 + tx * 4);
-    c[r][0] = lo.x; c[r][1] = lo.y; c[r][2] = lo.z; c[r][3] = lo.w;
-    c[r][4] = hi.x; c[r][5] = hi.y; c[r][6] = hi.z; c[r][7] = hi.w;
-  }
-  // row 0 is owned by ty = 0, r = 0
-  if (ty == 0) {
-    *reinterpret_cast<int4 *>(&rowbuf[0][tx * 4]) = make_int4(c[0][0], c[0][1], c[0][2], c[0][3]);
-    *reinterpret_cast<int4 *>(&rowbuf[0][64 + tx * 4]) = make_int4(c[0][4], c[0][5], c[0][6], c[0][7]);
-  }
-  __syncthreads();
-  for (int kk = 0; kk < TILE; ++kk) {
-    const int32_t *rb = rowbuf[kk & 1];
-    const int4 alo = *reinterpret_cast<const int4 *>(rb + ty * 4);
-    const int4 ahi = *reinterpret_cast<const int4 *>(rb + 64 + ty * 4);
-    const int4 blo = *reinterpret_cast<const int4 *>(rb + tx * 4);
-    const int4 bhi = *reinterpret_cast<const int4 *>(rb + 64 + tx * 4);
-    const int32_t a[8] = {alo.x, alo.y, alo.z, alo.w, ahi.x, ahi.y, ahi.z, ahi.w};
-    const int32_t b[8] = {blo.x, blo.y, blo.z, blo.w, bhi.x, bhi.y, bhi.z, bhi.w};
-#pragma unroll
-    for (int r = 0; r < 8; ++r)
-#pragma unroll
-      for (int q = 0; q < 8; ++q) c[r][q] = mp(a[r], b[q], c[r][q]);
-    // publish row kk+1 (after this step's update) for the next step
-    const int nk = kk + 1;
-    if (nk < TILE && ty == ((nk & 63) >> 2)) {
-      const int rr = (nk & 3) + (nk >= 64 ? 4 : 0);
-      int32_t *wb = rowbuf[nk & 1];
-#pragma unroll
-      for (int r = 0; r < 8; ++r) {
-        if (r == rr) {
-          *reinterpret_cast<int4 *>(wb + tx * 4) = make_int4(c[r][0], c[r][1], c[r][2], c[r][3]);
-          *reinterpret_cast<int4 *>(wb + 64 + tx * 4) = make_int4(c[r][4], c[r][5], c[r][6], c[r][7]);
-        }
-      }
-    }
-    __syncthreads();
-  }
-#pragma unroll
-  for (int r = 0; r < 8; ++r) {
-    const int i = (r < 4 ? 0 : 64) + ty * 4 + (r & 3);
-    *reinterpret_cast<int4 *>(T + (int64_t)i * ldt + tx * 4) = make_int4(c[r][0], c[r][1], c[r][2], c[r][3]);
-    *reinterpret_cast<int4 *>(T + (int64_t)i * ldt + 64 + tx * 4) = make_int4(c[r][4], c[r][5], c[r][6], c[r][7]);
-  }
-}
-
-// ------------------------------------------------------------------------------ phases 2 and 3
-// Persistent, TMA-fed min-plus tile kernel.  Each CTA walks its tiles (blockIdx.x, +gridDim.x, ...);
-// the operand chunks (A^T = P[k-rows][ti cols], B = P[k-rows][tj cols], 32 x 128 int32 each) stream
-// through a STAGES-deep shared-memory ring filled by cp.async.bulk.tensor (TMA) and guarded by
-// mbarriers (full: TMA bytes landed; empty: all 8 warps done reading), so no CTA-wide barrier sits
-// in the main loop and the next tile's first chunks are fetched while the current tile finishes.
-// Thread 0 doubles as the TMA producer.  The C tile lives in registers (8x8 per thread).
-// MODE_CROSS / MODE_REST (single-GPU lookahead, round k): the upper tiles of row/column k+1 (without
-// column k), and all upper tiles outside rows/columns k and k+1; together they are MODE_UPPER.
-// MODE_LIST_CROSS / MODE_LIST_REST: the same split of a rank's MODE_LIST tiles (sharded lookahead).
-// MODE_PIECES: phase 2 on the pivot-row pieces a rank contributes (owner-side phase 2, sharded FW):
-// tiles (k, orow[i]) for the mk owned rows above k, then (k, k+1 ..) when the rank owns row k (posk).
-enum { MODE_PIVOT_ROW = 0, MODE_UPPER = 1, MODE_LIST = 2, MODE_CROSS = 3, MODE_REST = 4, MODE_LIST_CROSS = 5,
-       MODE_LIST_REST = 6, MODE_PIECES = 7 };
-
-// Tile-kernel configuration: k-chunk depth, TMA ring depth, CTAs per SM, kk-loop unroll.
-template <int KC_, int ST_, int MINB_, int UNR_>
-struct FwCfg {
-  static constexpr int KC = KC_;
-  static constexpr int NCHUNK = TILE / KC_;
-  static constexpr int SM_CHUNK = KC_ * TILE;          // ints per operand chunk
-  static constexpr int STAGES = ST_;
-  static constexpr int MINB = MINB_;
-  static constexpr int UNR = UNR_;
-  static constexpr int SMEM = STAGES * 2 * SM_CHUNK * 4 + 2 * STAGES * 8;
-};
-
-struct TileJob {
-  int32_t *C;        // matrix holding the C tiles (local rows), leading dimension ldc
-  int64_t ldc;
-  int32_t p_row0;    // row coordinate of the pivot row block inside the operand tensor map
-  int32_t k;         // pivot tile index
-  int32_t nt;        // tiles per dimension (Np / 128)
-  int32_t ti0;       // first local tile row (global index) of C
-  int32_t nti;       // number of local tile rows
-  int32_t mode;
-  int32_t mirror;    // also write the transposed result into tile (tj, ti) (single GPU)
-  int64_t ntiles;    // tiles in this launch
-  // MODE_LIST (row-block sharded): the rank's owned tile rows (ascending), the static prefix sums of
-  // their upper-tile counts (nt - ti), and per round k: mk = #owned rows < k, posk = position of row k
-  // in the owned list or -1
-  const int32_t *orow;
-  const int64_t *opre;
-  int32_t nown, mk, posk;
-  int32_t posk1;     // MODE_LIST_CROSS / _REST: position of row k+1 in the owned list or -1
-};
-
+// ------------------------------------------------------------------------------ mbarrier / TMA
 __device__ __forceinline__ uint32_t smem_u32(const void *p) { return (uint32_t)__cvta_generic_to_shared(p); }
-
 __device__ __forceinline__ void mbar_init(uint64_t *b, uint32_t cnt) {
   asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;\n" ::"r"(smem_u32(b)), "r"(cnt) : "memory");
 }
@@ -181,20 +85,6 @@ __device__ __forceinline__ void mbar_wait(uint64_t *b, uint32_t parity) {
   while (!mbar_try(b, parity)) {
   }
 }
-// non-suspending poll (test_wait): the warp stays resident and issuing while it waits
-__device__ __forceinline__ bool mbar_test(uint64_t *b, uint32_t parity) {
-  uint32_t ok;
-  asm volatile(
-      "{\n\t.reg .pred p;\n\tmbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\n\tselp.u32 %0, 1, 0, p;\n\t}\n"
-      : "=r"(ok)
-      : "r"(smem_u32(b)), "r"(parity)
-      : "memory");
-  return ok != 0;
-}
-__device__ __forceinline__ void mbar_wait_spin(uint64_t *b, uint32_t parity) {
-  while (!mbar_test(b, parity)) {
-  }
-}
 __device__ __forceinline__ void tma_load_2d(void *dst, const CUtensorMap *map, int32_t c0, int32_t c1, uint64_t *bar) {
   asm volatile(
       "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];\n" ::"r"(
@@ -203,14 +93,163 @@ __device__ __forceinline__ void tma_load_2d(void *dst, const CUtensorMap *map, i
       : "memory");
 }
 
-__device__ __forceinline__ void tma_load_2d_hint(void *dst, const CUtensorMap *map, int32_t c0, int32_t c1, uint64_t *bar,
-                                                 uint64_t policy) {
-  asm volatile(
-      "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1, {%2, %3}], [%4], %5;\n" ::"r"(
-          smem_u32(dst)),
-      "l"(reinterpret_cast<uint64_t>(map)), "r"(c0), "r"(c1), "r"(smem_u32(bar)), "l"(policy)
-      : "memory");
+// ------------------------------------------------------------------------------ phase 1
+// Closure of the int32 128x128 pivot tile at T (leading dimension ldt), in place.
+__global__ void __launch_bounds__(NT, 1) k_fw_phase1(int32_t *T, int64_t ldt) {
+  __shared__ __align__(16) int32_t rowbuf[2][TILE];
+  const int tx = threadIdx.x & 15, ty = threadIdx.x >> 4;
+  int32_t c[8][8];
+#pragma unroll
+  for (int r = 0; r < 8; ++r) {
+    const int i = (r < 4 ? 0 : 64) + ty * 4 + (r & 3);
+    const int4 lo = *reinterpret_cast<const int4 *>(T + (int64_t)i * ldt + tx * 4);
+    const int4 hi = *reinterpret_cast<const int4 *>(T + (int64_t)i * ldt + 64 + tx * 4);
+    c[r][0] = lo.x; c[r][1] = lo.y; c[r][2] = lo.z; c[r][3] = lo.w;
+    c[r][4] = hi.x; c[r][5] = hi.y; c[r][6] = hi.z; c[r][7] = hi.w;
+  }
+  if (ty == 0) {   // row 0 is owned by ty = 0, r = 0
+    *reinterpret_cast<int4 *>(&rowbuf[0][tx * 4]) = make_int4(c[0][0], c[0][1], c[0][2], c[0][3]);
+    *reinterpret_cast<int4 *>(&rowbuf[0][64 + tx * 4]) = make_int4(c[0][4], c[0][5], c[0][6], c[0][7]);
+  }
+  __syncthreads();
+  for (int kk = 0; kk < TILE; ++kk) {
+    const int32_t *rb = rowbuf[kk & 1];
+    const int4 alo = *reinterpret_cast<const int4 *>(rb + ty * 4);
+    const int4 ahi = *reinterpret_cast<const int4 *>(rb + 64 + ty * 4);
+    const int4 blo = *reinterpret_cast<const int4 *>(rb + tx * 4);
+    const int4 bhi = *reinterpret_cast<const int4 *>(rb + 64 + tx * 4);
+    const int32_t a[8] = {alo.x, alo.y, alo.z, alo.w, ahi.x, ahi.y, ahi.z, ahi.w};
+    const int32_t b[8] = {blo.x, blo.y, blo.z, blo.w, bhi.x, bhi.y, bhi.z, bhi.w};
+#pragma unroll
+    for (int r = 0; r < 8; ++r)
+#pragma unroll
+      for (int q = 0; q < 8; ++q) c[r][q] = mp(a[r], b[q], c[r][q]);
+    const int nk = kk + 1;   // its owner publishes row nk (after this step's update) for the next step
+    if (nk < TILE && ty == ((nk & 63) >> 2)) {
+      const int rr = (nk & 3) + (nk >= 64 ? 4 : 0);
+      int32_t *wb = rowbuf[nk & 1];
+#pragma unroll
+      for (int r = 0; r < 8; ++r) {
+        if (r == rr) {
+          *reinterpret_cast<int4 *>(wb + tx * 4) = make_int4(c[r][0], c[r][1], c[r][2], c[r][3]);
+          *reinterpret_cast<int4 *>(wb + 64 + tx * 4) = make_int4(c[r][4], c[r][5], c[r][6], c[r][7]);
+        }
+      }
+    }
+    __syncthreads();
+  }
+#pragma unroll
+  for (int r = 0; r < 8; ++r) {
+    const int i = (r < 4 ? 0 : 64) + ty * 4 + (r & 3);
+    *reinterpret_cast<int4 *>(T + (int64_t)i * ldt + tx * 4) = make_int4(c[r][0], c[r][1], c[r][2], c[r][3]);
+    *reinterpret_cast<int4 *>(T + (int64_t)i * ldt + 64 + tx * 4) = make_int4(c[r][4], c[r][5], c[r][6], c[r][7]);
+  }
 }
+
+// Closure of the 16-bit pivot tile (ld ldt) in place, packed like the tile kernel: thread (ty, tx) owns
+// rows {ty*4 .. +3, 64 + ty*4 .. +3} as 4 row PAIRS and columns {tx*4 .. +3, 64 + tx*4 .. +3},
+// c[p][q] = (T[i][j], T[i+1][j]); step kk reads row kk from shared memory -- it is also column kk, the
+// tile being symmetric -- as the row-pair operand and, duplicated, as the column operand, so one
+// VIADDMNMX.U16x2 relaxes two entries (values <= C16: sums <= 0xFFFE never wrap, results stay <= C16).
+// About 60 registers: it fits beside the tile kernel's CTAs, which the lookahead needs.
+__global__ void __launch_bounds__(NT, 1) k_fw_phase1_16(uint16_t *T, int64_t ldt) {
+  __shared__ __align__(16) uint16_t rowbuf[2][TILE];
+  const int tx = threadIdx.x & 15, ty = threadIdx.x >> 4;
+  uint32_t c[4][8];
+#pragma unroll
+  for (int p = 0; p < 4; ++p) {
+    const int i = (p < 2 ? 0 : 64) + ty * 4 + (p & 1) * 2;
+#pragma unroll
+    for (int h = 0; h < 2; ++h) {
+      const uint2 v = *reinterpret_cast<const uint2 *>(T + (int64_t)i * ldt + h * 64 + tx * 4);
+      const uint2 w = *reinterpret_cast<const uint2 *>(T + (int64_t)(i + 1) * ldt + h * 64 + tx * 4);
+      c[p][h * 4 + 0] = __byte_perm(v.x, w.x, 0x5410);
+      c[p][h * 4 + 1] = __byte_perm(v.x, w.x, 0x7632);
+      c[p][h * 4 + 2] = __byte_perm(v.y, w.y, 0x5410);
+      c[p][h * 4 + 3] = __byte_perm(v.y, w.y, 0x7632);
+    }
+  }
+  if (threadIdx.x < TILE / 4)   // row 0
+    reinterpret_cast<uint2 *>(rowbuf[0])[threadIdx.x] = reinterpret_cast<const uint2 *>(T)[threadIdx.x];
+  __syncthreads();
+  for (int kk = 0; kk < TILE; ++kk) {
+    const uint16_t *rb = rowbuf[kk & 1];
+    const uint2 alo = *reinterpret_cast<const uint2 *>(rb + ty * 4);
+    const uint2 ahi = *reinterpret_cast<const uint2 *>(rb + 64 + ty * 4);
+    const uint2 blo = *reinterpret_cast<const uint2 *>(rb + tx * 4);
+    const uint2 bhi = *reinterpret_cast<const uint2 *>(rb + 64 + tx * 4);
+    const uint32_t a[4] = {alo.x, alo.y, ahi.x, ahi.y};
+    const uint32_t b[8] = {__byte_perm(blo.x, 0, 0x1010), __byte_perm(blo.x, 0, 0x3232),
+                           __byte_perm(blo.y, 0, 0x1010), __byte_perm(blo.y, 0, 0x3232),
+                           __byte_perm(bhi.x, 0, 0x1010), __byte_perm(bhi.x, 0, 0x3232),
+                           __byte_perm(bhi.y, 0, 0x1010), __byte_perm(bhi.y, 0, 0x3232)};
+#pragma unroll
+    for (int p = 0; p < 4; ++p)
+#pragma unroll
+      for (int q = 0; q < 8; ++q) c[p][q] = __viaddmin_u16x2(a[p], b[q], c[p][q]);
+    const int nk = kk + 1;
+    if (nk < TILE && ty == ((nk & 63) >> 2)) {
+      const int p = ((nk & 3) >> 1) + (nk >= 64 ? 2 : 0), hi = nk & 1;
+      uint16_t *wb = rowbuf[nk & 1];
+#pragma unroll
+      for (int pp = 0; pp < 4; ++pp) {
+        if (pp == p) {
+          const uint32_t sel = hi ? 0x7632 : 0x5410;
+          *reinterpret_cast<uint2 *>(wb + tx * 4) =
+              make_uint2(__byte_perm(c[pp][0], c[pp][1], sel), __byte_perm(c[pp][2], c[pp][3], sel));
+          *reinterpret_cast<uint2 *>(wb + 64 + tx * 4) =
+              make_uint2(__byte_perm(c[pp][4], c[pp][5], sel), __byte_perm(c[pp][6], c[pp][7], sel));
+        }
+      }
+    }
+    __syncthreads();
+  }
+#pragma unroll
+  for (int p = 0; p < 4; ++p) {
+    const int i = (p < 2 ? 0 : 64) + ty * 4 + (p & 1) * 2;
+#pragma unroll
+    for (int h = 0; h < 2; ++h) {
+      const uint32_t *cc = &c[p][h * 4];
+      *reinterpret_cast<uint2 *>(T + (int64_t)i * ldt + h * 64 + tx * 4) =
+          make_uint2(__byte_perm(cc[0], cc[1], 0x5410), __byte_perm(cc[2], cc[3], 0x5410));
+      *reinterpret_cast<uint2 *>(T + (int64_t)(i + 1) * ldt + h * 64 + tx * 4) =
+          make_uint2(__byte_perm(cc[0], cc[1], 0x7632), __byte_perm(cc[2], cc[3], 0x7632));
+    }
+  }
+}
+
+// ------------------------------------------------------------------------------ phases 2 and 3
+// Tile sets of one launch (round k):
+//   MODE_PIVOT_ROW   tiles (k, j != k)                        -- phase 2, single GPU
+//   MODE_UPPER       upper tiles outside row/column k         -- phase 3, single GPU
+//   MODE_CROSS       upper tiles of row/column k+1 (not k)    -- lookahead: first part of phase 3
+//   MODE_REST        upper tiles outside rows/columns k, k+1  -- lookahead: the rest
+//   MODE_LIST        a rank's owned upper tiles outside row/column k (C addressed by local tile row)
+//   MODE_LIST_CROSS / MODE_LIST_REST   the same split of MODE_LIST
+//   MODE_PIECES      phase 2 on the pivot-row pieces a rank contributes: tiles (k, orow[i]) for its mk
+//                    owned rows above k, then (k, k+1 ..) when it owns row k (posk >= 0)
+enum { MODE_PIVOT_ROW = 0, MODE_UPPER = 1, MODE_LIST = 2, MODE_CROSS = 3, MODE_REST = 4, MODE_LIST_CROSS = 5,
+       MODE_LIST_REST = 6, MODE_PIECES = 7 };
+
+struct TileJob {
+  void *C;           // matrix holding the C tiles (local tile rows), leading dimension ldc (elements)
+  int64_t ldc;
+  int32_t a_row0;    // row of the pivot row block inside the A operand's tensor map
+  int32_t b_row0;    // ... inside the B operand's map
+  int32_t k;         // pivot tile index
+  int32_t nt;        // tiles per dimension (Np / 128)
+  int32_t ti0;       // first tile row held by C (lr = ti - ti0 outside the list modes)
+  int32_t mode;
+  int32_t mirror;    // also write the transposed result into tile (tj, ti) (single GPU)
+  int64_t ntiles;    // tiles in this launch
+  // list modes: the rank's owned tile rows (ascending), the static prefix sums of their upper-tile
+  // counts (nt - ti), and per round: mk = #owned rows < k, posk / posk1 = position of row k / k+1 in
+  // the owned list or -1
+  const int32_t *orow;
+  const int64_t *opre;
+  int32_t nown, mk, posk, posk1;
+  int32_t *counter;  // {next tile, CTAs done}: zero at launch, reset by the launch's last CTA
+};
 
 // decode the tile index into (ti, tj) and the local tile row lr of C
 __device__ __forceinline__ void decode_tile(const TileJob &J, int64_t idx, int &ti, int &tj, int &lr) {
@@ -280,193 +319,242 @@ __device__ __forceinline__ void decode_tile(const TileJob &J, int64_t idx, int &
   if (ti < k && tj >= k) tj += rest ? 2 : 1;
 }
 
-template <class CF>
-__global__ void __launch_bounds__(NT, CF::MINB) k_fw_tiles(const __grid_constant__ CUtensorMap tmP, const TileJob J) {
-  constexpr int KC = CF::KC, NCHUNK = CF::NCHUNK, SM_CHUNK = CF::SM_CHUNK, STAGES = CF::STAGES;
-  extern __shared__ __align__(128) int32_t smem[];
-  int32_t *sA = smem;                                   // [STAGES][KC][TILE]  A^T chunks
-  int32_t *sB = sA + STAGES * SM_CHUNK;                 // [STAGES][KC][TILE]  B chunks
-  uint64_t *full = reinterpret_cast<uint64_t *>(sB + STAGES * SM_CHUNK);
-  uint64_t *empty = full + STAGES;
-  const int tid = threadIdx.x, lane = tid & 31;
-  const int tx = tid & 15, ty = tid >> 4;
-
-  const int my_tiles = J.ntiles > (int64_t)blockIdx.x ? (int)((J.ntiles - 1 - blockIdx.x) / gridDim.x + 1) : 0;
-  const int total_chunks = my_tiles * NCHUNK;
-  int issued = 0;   // producer state (thread 0 only)
-  auto tile_of = [&](int it, int &ti, int &tj, int &lr) {
-    decode_tile(J, blockIdx.x + (int64_t)it * gridDim.x, ti, tj, lr);
+// Fragment policies of the tile kernel: C tile in registers, operand chunks (KC rows of the pivot row
+// block, A^T for the tile's rows, B for its columns) from shared memory.
+//
+// Frag32: 256 threads, 8 x 8 int32 per thread (rows {ty*4 .. +3, 64 + ty*4 .. +3}, columns
+// {tx*4 .. +3, 64 + tx*4 .. +3}), 64-deep chunks, 2-stage ring (128 KB), one CTA per SM: chosen by
+// measurement on the B200 (round 1, profiles/r01_fw_variants.txt: 88 % of the int32 VIADDMNMX peak).
+struct Frag32 {
+  using E = int32_t;
+  static constexpr int NTH = 256, KC = 64, STAGES = 2, MINB = 1;
+  static constexpr int A_BYTES = KC * TILE * 4, B_BYTES = KC * TILE * 4;
+  struct Acc {
+    int32_t c[8][8];
   };
-  auto produce = [&](int upto) {
-    while (issued < upto) {
-      const int st = issued % STAGES;
-      if (issued >= STAGES) mbar_wait(&empty[st], (uint32_t)((issued / STAGES - 1) & 1));
-      int pti, ptj, plr;
-      tile_of(issued / NCHUNK, pti, ptj, plr);
-      const int row = J.p_row0 + (issued % NCHUNK) * KC;
-      mbar_arrive_tx(&full[st], 2 * SM_CHUNK * 4);
-      tma_load_2d(sA + st * SM_CHUNK, &tmP, pti * TILE, row, &full[st]);
-      tma_load_2d(sB + st * SM_CHUNK, &tmP, ptj * TILE, row, &full[st]);
-      ++issued;
+  __device__ static int row(int r, int ty) { return (r < 4 ? 0 : 64) + ty * 4 + (r & 3); }
+  __device__ static void load(Acc &a, const E *Ct, int64_t ldc, int tid) {
+    const int tx = tid & 15, ty = tid >> 4;
+#pragma unroll
+    for (int r = 0; r < 8; ++r) {
+      const int i = row(r, ty);
+      const int4 lo = *reinterpret_cast<const int4 *>(Ct + (int64_t)i * ldc + tx * 4);
+      const int4 hi = *reinterpret_cast<const int4 *>(Ct + (int64_t)i * ldc + 64 + tx * 4);
+      a.c[r][0] = lo.x; a.c[r][1] = lo.y; a.c[r][2] = lo.z; a.c[r][3] = lo.w;
+      a.c[r][4] = hi.x; a.c[r][5] = hi.y; a.c[r][6] = hi.z; a.c[r][7] = hi.w;
     }
-  };
+  }
+  __device__ static void chunk(Acc &a, const uint8_t *sa, const uint8_t *sb, int tid) {
+    const int tx = tid & 15, ty = tid >> 4;
+    const int32_t *a_s = reinterpret_cast<const int32_t *>(sa), *b_s = reinterpret_cast<const int32_t *>(sb);
+#pragma unroll 16
+    for (int kk = 0; kk < KC; ++kk) {
+      const int4 alo = *reinterpret_cast<const int4 *>(a_s + kk * TILE + ty * 4);
+      const int4 ahi = *reinterpret_cast<const int4 *>(a_s + kk * TILE + 64 + ty * 4);
+      const int4 blo = *reinterpret_cast<const int4 *>(b_s + kk * TILE + tx * 4);
+      const int4 bhi = *reinterpret_cast<const int4 *>(b_s + kk * TILE + 64 + tx * 4);
+      const int32_t av[8] = {alo.x, alo.y, alo.z, alo.w, ahi.x, ahi.y, ahi.z, ahi.w};
+      const int32_t bv[8] = {blo.x, blo.y, blo.z, blo.w, bhi.x, bhi.y, bhi.z, bhi.w};
+#pragma unroll
+      for (int r = 0; r < 8; ++r)
+#pragma unroll
+        for (int q = 0; q < 8; ++q) a.c[r][q] = mp(av[r], bv[q], a.c[r][q]);
+    }
+  }
+  __device__ static void store(const Acc &a, E *Ct, int64_t ldc, int tid) {
+    const int tx = tid & 15, ty = tid >> 4;
+#pragma unroll
+    for (int r = 0; r < 8; ++r) {
+      const int i = row(r, ty);
+      *reinterpret_cast<int4 *>(Ct + (int64_t)i * ldc + tx * 4) = make_int4(a.c[r][0], a.c[r][1], a.c[r][2], a.c[r][3]);
+      *reinterpret_cast<int4 *>(Ct + (int64_t)i * ldc + 64 + tx * 4) = make_int4(a.c[r][4], a.c[r][5], a.c[r][6], a.c[r][7]);
+    }
+  }
+  __device__ static void store_mirror(const Acc &a, E *Mt, int64_t ldc, int tid) {
+    const int tx = tid & 15, ty = tid >> 4;
+#pragma unroll
+    for (int q = 0; q < 8; ++q) {
+      const int j = (q < 4 ? 0 : 64) + tx * 4 + (q & 3);
+      *reinterpret_cast<int4 *>(Mt + (int64_t)j * ldc + ty * 4) = make_int4(a.c[0][q], a.c[1][q], a.c[2][q], a.c[3][q]);
+      *reinterpret_cast<int4 *>(Mt + (int64_t)j * ldc + 64 + ty * 4) = make_int4(a.c[4][q], a.c[5][q], a.c[6][q], a.c[7][q]);
+    }
+  }
+};
 
+// Frag16: 128 threads, 16 rows x 8 columns each as 8 row PAIRS x 8 columns, c[p][q] = (C[i][j], C[i+1][j])
+// packed; A chunks are u16 rows of the pivot row block (row pairs are adjacent u16: one register), B
+// chunks rows of its copy with every value duplicated into both halves, so one VIADDMNMX.U16x2 updates
+// two entries with no unpacking in the inner loop.  32-deep chunks, 2-stage ring (48 KB), 3 CTAs per
+// SM: chosen by a 17-variant sweep on the B200 (round 1, profiles/r01_fw16_variants.jsonl).
+struct Frag16 {
+  using E = uint16_t;
+  static constexpr int NTH = 128, KC = 32, STAGES = 2, MINB = 3;
+  static constexpr int A_BYTES = KC * TILE * 2, B_BYTES = KC * TILE * 4;
+  struct Acc {
+    uint32_t c[8][8];
+  };
+  __device__ static int row(int r2, int ty) { return (r2 < 4 ? 0 : 64) + ty * 8 + (r2 & 3) * 2; }
+  __device__ static void load(Acc &a, const E *Ct, int64_t ldc, int tid) {
+    const int tx = tid & 15, ty = tid >> 4;
+#pragma unroll
+    for (int r2 = 0; r2 < 8; ++r2) {
+      const int i = row(r2, ty);
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        const uint2 v = *reinterpret_cast<const uint2 *>(Ct + (int64_t)i * ldc + h * 64 + tx * 4);
+        const uint2 w = *reinterpret_cast<const uint2 *>(Ct + (int64_t)(i + 1) * ldc + h * 64 + tx * 4);
+        a.c[r2][h * 4 + 0] = __byte_perm(v.x, w.x, 0x5410);
+        a.c[r2][h * 4 + 1] = __byte_perm(v.x, w.x, 0x7632);
+        a.c[r2][h * 4 + 2] = __byte_perm(v.y, w.y, 0x5410);
+        a.c[r2][h * 4 + 3] = __byte_perm(v.y, w.y, 0x7632);
+      }
+    }
+  }
+  __device__ static void chunk(Acc &a, const uint8_t *sa, const uint8_t *sb, int tid) {
+    const int tx = tid & 15, ty = tid >> 4;
+    const uint16_t *a_s = reinterpret_cast<const uint16_t *>(sa);
+    const uint32_t *b_s = reinterpret_cast<const uint32_t *>(sb);
+#pragma unroll 16
+    for (int kk = 0; kk < KC; ++kk) {
+      const uint4 alo = *reinterpret_cast<const uint4 *>(a_s + kk * TILE + ty * 8);
+      const uint4 ahi = *reinterpret_cast<const uint4 *>(a_s + kk * TILE + 64 + ty * 8);
+      const uint32_t av[8] = {alo.x, alo.y, alo.z, alo.w, ahi.x, ahi.y, ahi.z, ahi.w};
+      const uint4 blo = *reinterpret_cast<const uint4 *>(b_s + kk * TILE + tx * 4);
+      const uint4 bhi = *reinterpret_cast<const uint4 *>(b_s + kk * TILE + 64 + tx * 4);
+      const uint32_t bv[8] = {blo.x, blo.y, blo.z, blo.w, bhi.x, bhi.y, bhi.z, bhi.w};
+#pragma unroll
+      for (int r2 = 0; r2 < 8; ++r2)
+#pragma unroll
+        for (int q = 0; q < 8; ++q) a.c[r2][q] = __viaddmin_u16x2(av[r2], bv[q], a.c[r2][q]);
+    }
+  }
+  __device__ static void store(const Acc &a, E *Ct, int64_t ldc, int tid) {
+    const int tx = tid & 15, ty = tid >> 4;
+#pragma unroll
+    for (int r2 = 0; r2 < 8; ++r2) {
+      const int i = row(r2, ty);
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        const uint32_t *cc = &a.c[r2][h * 4];
+        *reinterpret_cast<uint2 *>(Ct + (int64_t)i * ldc + h * 64 + tx * 4) =
+            make_uint2(__byte_perm(cc[0], cc[1], 0x5410), __byte_perm(cc[2], cc[3], 0x5410));
+        *reinterpret_cast<uint2 *>(Ct + (int64_t)(i + 1) * ldc + h * 64 + tx * 4) =
+            make_uint2(__byte_perm(cc[0], cc[1], 0x7632), __byte_perm(cc[2], cc[3], 0x7632));
+      }
+    }
+  }
+  __device__ static void store_mirror(const Acc &a, E *Mt, int64_t ldc, int tid) {
+    const int tx = tid & 15, ty = tid >> 4;
+#pragma unroll
+    for (int q = 0; q < 8; ++q) {
+      const int j = (q < 4 ? 0 : 64) + tx * 4 + (q & 3);
+#pragma unroll
+      for (int h = 0; h < 2; ++h)
+        *reinterpret_cast<uint4 *>(Mt + (int64_t)j * ldc + h * 64 + ty * 8) =
+            make_uint4(a.c[h * 4][q], a.c[h * 4 + 1][q], a.c[h * 4 + 2][q], a.c[h * 4 + 3][q]);
+    }
+  }
+};
+
+// The tile kernel.  Persistent CTAs, dynamically scheduled: a CTA takes its next tile from a global
+// counter when it issues that tile's first TMA chunk (round 1 measured the static assignment ending
+// its CTAs between 43 % and 100 % of a launch -- the CTAs of an SM run at different speeds), and
+// publishes it, tagged with its sequence number q, in tslot[q & 1]; the ring depth (2) never exceeds
+// the chunks per tile, so a slot is rewritten only after every warp has read it.  Operand chunks
+// stream through a STAGES-deep shared-memory ring filled by cp.async.bulk.tensor (TMA), completion
+// tracked by mbarriers; a stage is refilled by the LAST warp to finish reading it (a shared counter),
+// so no CTA-wide barrier sits in the main loop.  The last CTA to finish resets the counter pair.
+template <class F>
+__global__ void __launch_bounds__(F::NTH, F::MINB)
+    k_fw_tiles(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB, const TileJob J) {
+  constexpr int KC = F::KC, NCHUNK = TILE / KC, STAGES = F::STAGES, NW = F::NTH / 32;
+  static_assert(NCHUNK >= STAGES, "tile slots are rewritten only after every warp has read them");
+  constexpr int32_t NONE = 0xFFFFF;
+  using E = typename F::E;
+  extern __shared__ __align__(128) uint8_t smem[];
+  uint8_t *sA = smem;
+  uint8_t *sB = sA + STAGES * F::A_BYTES;
+  uint64_t *full = reinterpret_cast<uint64_t *>(sB + STAGES * F::B_BYTES);
+  int32_t *cnt = reinterpret_cast<int32_t *>(full + STAGES);   // [STAGES] warps done with the stage
+  int32_t *tslot = cnt + STAGES;                               // [2] (q << 20) | tile
+  const int tid = threadIdx.x, lane = tid & 31;
+  auto issue = [&](int c, int st) {   // chunk c of this CTA's sequence into stage st (one thread)
+    const int q = c / NCHUNK, kc = c % NCHUNK;
+    int32_t t;
+    if (kc == 0) {
+      const int32_t tt = atomicAdd(J.counter, 1);
+      t = tt < J.ntiles ? tt : -1;
+      tslot[q & 1] = (q << 20) | (t < 0 ? NONE : t);
+      __threadfence_block();
+    } else {
+      const int32_t v = tslot[q & 1] & NONE;
+      t = v == NONE ? -1 : v;
+    }
+    if (t < 0) {   // no tile: complete the phase without data so that the waiters see the end
+      mbar_arrive(&full[st]);
+      return;
+    }
+    int pti, ptj, plr;
+    decode_tile(J, t, pti, ptj, plr);
+    mbar_arrive_tx(&full[st], F::A_BYTES + F::B_BYTES);
+    tma_load_2d(sA + st * F::A_BYTES, &tmA, pti * TILE, J.a_row0 + kc * KC, &full[st]);
+    tma_load_2d(sB + st * F::B_BYTES, &tmB, ptj * TILE, J.b_row0 + kc * KC, &full[st]);
+  };
   if (tid == 0) {
     for (int s = 0; s < STAGES; ++s) {
       mbar_init(&full[s], 1);
-      mbar_init(&empty[s], NT / 32);
+      cnt[s] = 0;
     }
     asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
-    asm volatile("prefetch.tensormap [%0];\n" ::"l"(reinterpret_cast<uint64_t>(&tmP)) : "memory");
+    asm volatile("prefetch.tensormap [%0];\n" ::"l"(reinterpret_cast<uint64_t>(&tmA)) : "memory");
+    asm volatile("prefetch.tensormap [%0];\n" ::"l"(reinterpret_cast<uint64_t>(&tmB)) : "memory");
   }
   __syncthreads();
-  if (tid == 0 && my_tiles > 0) produce(total_chunks < STAGES ? total_chunks : STAGES);
+  if (tid == 0)
+    for (int c = 0; c < STAGES; ++c) issue(c, c);
 
-  int g = 0;   // chunk counter (all threads)
-  for (int it = 0; it < my_tiles; ++it) {
+  int g = 0;
+  for (int q = 0;; ++q) {
+    mbar_wait(&full[g % STAGES], (uint32_t)((g / STAGES) & 1));
+    const int32_t v = tslot[q & 1] & NONE;
+    if (v == NONE) break;
     int ti, tj, lr;
-    tile_of(it, ti, tj, lr);
-    int32_t c[8][8];
-    // C tile straight from global memory into registers (its latency overlaps the in-flight TMA chunks)
-    int32_t *Ct = J.C + (int64_t)lr * TILE * J.ldc + (int64_t)tj * TILE;
-#pragma unroll
-    for (int r = 0; r < 8; ++r) {
-      const int i = (r < 4 ? 0 : 64) + ty * 4 + (r & 3);
-      const int4 lo = *reinterpret_cast<const int4 *>(Ct + (int64_t)i * J.ldc + tx * 4);
-      const int4 hi = *reinterpret_cast<const int4 *>(Ct + (int64_t)i * J.ldc + 64 + tx * 4);
-      c[r][0] = lo.x; c[r][1] = lo.y; c[r][2] = lo.z; c[r][3] = lo.w;
-      c[r][4] = hi.x; c[r][5] = hi.y; c[r][6] = hi.z; c[r][7] = hi.w;
-    }
+    decode_tile(J, v, ti, tj, lr);
+    E *Ct = static_cast<E *>(J.C) + (int64_t)lr * TILE * J.ldc + (int64_t)tj * TILE;
+    typename F::Acc acc;
+    F::load(acc, Ct, J.ldc, tid);   // C straight into registers (its latency overlaps the in-flight TMA)
 #pragma unroll 1
     for (int kc = 0; kc < NCHUNK; ++kc, ++g) {
-      if (tid == 0) produce(g + STAGES < total_chunks ? g + STAGES : total_chunks);
       const int st = g % STAGES;
-      mbar_wait(&full[st], (uint32_t)((g / STAGES) & 1));
-      const int32_t *a_s = sA + st * SM_CHUNK;
-      const int32_t *b_s = sB + st * SM_CHUNK;
-#pragma unroll CF::UNR
-      for (int kk = 0; kk < KC; ++kk) {
-        const int4 alo = *reinterpret_cast<const int4 *>(a_s + kk * TILE + ty * 4);
-        const int4 ahi = *reinterpret_cast<const int4 *>(a_s + kk * TILE + 64 + ty * 4);
-        const int4 blo = *reinterpret_cast<const int4 *>(b_s + kk * TILE + tx * 4);
-        const int4 bhi = *reinterpret_cast<const int4 *>(b_s + kk * TILE + 64 + tx * 4);
-        const int32_t a[8] = {alo.x, alo.y, alo.z, alo.w, ahi.x, ahi.y, ahi.z, ahi.w};
-        const int32_t b[8] = {blo.x, blo.y, blo.z, blo.w, bhi.x, bhi.y, bhi.z, bhi.w};
-#pragma unroll
-        for (int r = 0; r < 8; ++r)
-#pragma unroll
-          for (int q = 0; q < 8; ++q) c[r][q] = mp(a[r], b[q], c[r][q]);
-      }
+      if (kc > 0) mbar_wait(&full[st], (uint32_t)((g / STAGES) & 1));
+      F::chunk(acc, sA + st * F::A_BYTES, sB + st * F::B_BYTES, tid);
       __syncwarp();
-      if (lane == 0) mbar_arrive(&empty[st]);
-    }
-    // epilogue: tile, and (single GPU, off-diagonal) its transposed mirror
-#pragma unroll
-    for (int r = 0; r < 8; ++r) {
-      const int i = (r < 4 ? 0 : 64) + ty * 4 + (r & 3);
-      *reinterpret_cast<int4 *>(Ct + (int64_t)i * J.ldc + tx * 4) = make_int4(c[r][0], c[r][1], c[r][2], c[r][3]);
-      *reinterpret_cast<int4 *>(Ct + (int64_t)i * J.ldc + 64 + tx * 4) = make_int4(c[r][4], c[r][5], c[r][6], c[r][7]);
-    }
-    if (J.mirror && ti != tj) {
-      int32_t *Mt = J.C + (int64_t)tj * TILE * J.ldc + (int64_t)ti * TILE;
-#pragma unroll
-      for (int q = 0; q < 8; ++q) {
-        const int j = (q < 4 ? 0 : 64) + tx * 4 + (q & 3);
-        *reinterpret_cast<int4 *>(Mt + (int64_t)j * J.ldc + ty * 4) = make_int4(c[0][q], c[1][q], c[2][q], c[3][q]);
-        *reinterpret_cast<int4 *>(Mt + (int64_t)j * J.ldc + 64 + ty * 4) = make_int4(c[4][q], c[5][q], c[6][q], c[7][q]);
+      if (lane == 0) {
+        __threadfence_block();
+        if (atomicAdd(&cnt[st], 1) == NW - 1) {   // the last reader of this stage refills it
+          cnt[st] = 0;
+          __threadfence_block();
+          asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");
+          issue(g + STAGES, st);
+        }
       }
     }
+    F::store(acc, Ct, J.ldc, tid);
+    if (J.mirror && ti != tj)
+      F::store_mirror(acc, static_cast<E *>(J.C) + (int64_t)tj * TILE * J.ldc + (int64_t)ti * TILE, J.ldc, tid);
   }
-}
-
-__global__ void k_fill(int32_t *p, int64_t n, int32_t v) {
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) p[i] = v;
-}
-
-__global__ void k_fill16(uint16_t *p, int64_t n2, uint32_t v2) {   // n2 u16 pairs
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n2; i += (int64_t)gridDim.x * blockDim.x)
-    reinterpret_cast<uint32_t *>(p)[i] = v2;
-}
-
-// u16 block -> int32 (the values are capped 16-bit distances, C16 included), n % 4 == 0
-__global__ void k_widen16(const uint16_t *__restrict__ P16, int32_t *__restrict__ P32, int64_t n) {
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n / 4; i += (int64_t)gridDim.x * blockDim.x) {
-    const uint2 v = reinterpret_cast<const uint2 *>(P16)[i];
-    reinterpret_cast<int4 *>(P32)[i] = make_int4(v.x & 0xFFFF, v.x >> 16, v.y & 0xFFFF, v.y >> 16);
-  }
-}
-
-// Pivot-row block <-> a rank's owned storage, round k (prow: 128 x Np, leading dimension Np).
-//   dir = 0 (gather):  prow[:, ti-block] = S(ti, k)^T for owned ti < k; prow[:, j >= k] = S(k, j) if row k owned
-//   dir = 1 (scatter): the inverse, after phases 1 and 2 updated prow
-// Only the pieces are launched: grid (16 sub-blocks of 32 x 32, npieces), 256 threads, where pieces
-// [0, nrow) are the tiles j = k + y of the pivot row when this rank owns it (nrow = nt - k, local row
-// posk) and the next mk are the owned rows ti < k (the first mk owned rows: ascending), tile (ti, k).
-// TS / TP: storage / block element types (int32 <-> int32; u16 -> int32 to assemble the packed
-// schedule's exchange block, u16 -> u16 to scatter its narrowed block back).
-template <class TS, class TP>
-__global__ void k_prow_xfer(TS *S, int64_t ldd, const int32_t *orow, int32_t k, int32_t nt, int32_t posk, TP *prow,
-                            int32_t Np, int dir) {
-  __shared__ uint32_t t[32][33];
-  const int nrow = posk >= 0 ? nt - k : 0;
-  const int y = blockIdx.y;
-  const int bx = blockIdx.x & 3, by = blockIdx.x >> 2;         // 32 x 32 sub-block (bx: x, by: y)
-  const int lx = threadIdx.x & 31, ly = threadIdx.x >> 5;      // 32 x 8 threads
-  if (y < nrow) {              // the pivot row's upper part: plain copy, tiles j >= k
-    const int lr = posk, tj = k + y;
-    for (int yy = ly; yy < 32; yy += 8) {
-      const int64_t row = by * 32 + yy, col = (int64_t)tj * TILE + bx * 32 + lx;
-      TS *sp = S + ((int64_t)lr * TILE + row) * ldd + col;
-      TP *pp = prow + row * Np + col;
-      if (dir == 0) *pp = (TP)*sp; else *sp = (TS)*pp;
-    }
-    return;
-  }
-  const int lr = y - nrow, ti = orow[lr];   // owned row below the pivot: tile (ti, k) <-> prow[:, ti-block]^T
-  if (dir == 0) {
-    for (int yy = ly; yy < 32; yy += 8)   // S rows ti-block (bx*32+yy), cols k-block (by*32+lx)
-      t[yy][lx] = (uint32_t)S[((int64_t)lr * TILE + bx * 32 + yy) * ldd + (int64_t)k * TILE + by * 32 + lx];
-    __syncthreads();
-    for (int yy = ly; yy < 32; yy += 8)   // prow rows (by*32+yy), cols ti-block (bx*32+lx)
-      prow[(int64_t)(by * 32 + yy) * Np + (int64_t)ti * TILE + bx * 32 + lx] = (TP)t[lx][yy];
-  } else {
-    for (int yy = ly; yy < 32; yy += 8)
-      t[yy][lx] = (uint32_t)prow[(int64_t)(by * 32 + yy) * Np + (int64_t)ti * TILE + bx * 32 + lx];
-    __syncthreads();
-    for (int yy = ly; yy < 32; yy += 8)
-      S[((int64_t)lr * TILE + bx * 32 + yy) * ldd + (int64_t)k * TILE + by * 32 + lx] = (TS)t[lx][yy];
-  }
-}
-
-// owned upper tiles (ti, tj >= ti) -> full D, and their transposed mirrors (tj, ti)
-// grid: (16 sub-blocks, nt column tiles, nown owned rows), 256 threads
-__global__ void k_scatter_upper(const int32_t *S, int64_t ldd, const int32_t *orow, int32_t *Df, int64_t ldf) {
-  __shared__ int32_t t[32][33];
-  const int lr = blockIdx.z, ti = orow[lr], tj = blockIdx.y;
-  if (tj < ti) return;
-  const int bx = blockIdx.x & 3, by = blockIdx.x >> 2;
-  const int lx = threadIdx.x & 31, ly = threadIdx.x >> 5;
-  for (int yy = ly; yy < 32; yy += 8) {
-    const int32_t v = S[((int64_t)lr * TILE + by * 32 + yy) * ldd + (int64_t)tj * TILE + bx * 32 + lx];
-    Df[((int64_t)ti * TILE + by * 32 + yy) * ldf + (int64_t)tj * TILE + bx * 32 + lx] = v;
-    t[yy][lx] = v;
-  }
-  if (tj == ti) return;
   __syncthreads();
-  for (int yy = ly; yy < 32; yy += 8)
-    Df[((int64_t)tj * TILE + bx * 32 + yy) * ldf + (int64_t)ti * TILE + by * 32 + lx] = t[lx][yy];
+  if (tid == 0) {
+    __threadfence();
+    if (atomicAdd(J.counter + 1, 1) == (int)gridDim.x - 1) {   // the last CTA resets the pair
+      J.counter[0] = 0;
+      J.counter[1] = 0;
+      __threadfence();
+    }
+  }
 }
 
-// ------------------------------------------------------------------------------ 16-bit path
-// Packed unsigned 16-bit FW (VIADDMNMX.U16x2: two min-plus per instruction, twice the int32 issue
-// rate; microbench/minplus_peak.cu).  Values are capped at C16 = 0x7FFF: with a, b <= C16 the
-// 16-bit sum a + b <= 0xFFFE never wraps, and FW over capped values yields exactly min(d, C16) for
-// every pair (min(min(a,C)+min(b,C), C) = min(a+b, C) for a, b >= 0, so the cap commutes with every
-// relaxation).  Hence every entry < C16 is the exact distance; an entry == C16 is exact (unreachable)
-// iff its two vertices lie in different components -- checked afterwards, with a fall back to the
-// int32 FW on the untouched int32 D when some connected pair reached the cap.
-constexpr uint32_t C16 = 0x7FFF;
-
+// ------------------------------------------------------------------------------ 16-bit conversions
 __global__ void k_to16(const int32_t *__restrict__ D, int64_t ldd, uint16_t *__restrict__ D16, int32_t Np) {
   const int64_t total = (int64_t)Np * (Np / 4);
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
@@ -478,7 +566,7 @@ __global__ void k_to16(const int32_t *__restrict__ D, int64_t ldd, uint16_t *__r
   }
 }
 
-// capped entries of connected pairs (lab[i] == lab[j]; only vertices < n_real, labels may be null:
+// capped entries of connected pairs (lab[i] == lab[j]; only vertices < n_real; labels may be null:
 // then [0, n_real) is one component) -> *bad
 __global__ void k_check16(const uint16_t *__restrict__ D16, int32_t Np, const int32_t *__restrict__ lab, int32_t n_real,
                           int32_t *bad) {
@@ -499,7 +587,7 @@ __global__ void k_check16(const uint16_t *__restrict__ D16, int32_t Np, const in
   if (__syncthreads_or(found) && threadIdx.x == 0) atomicOr(bad, 1);
 }
 
-// largest finite entry of a distance row (the cap precheck of fw_single16)
+// largest finite entry of a distance row (the cap precheck)
 __global__ void k_row_far(const int32_t *__restrict__ row, int32_t n, int32_t *far) {
   int32_t m = 0;
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
@@ -521,7 +609,7 @@ __global__ void k_from16(const uint16_t *__restrict__ D16, int32_t Np, int32_t *
   }
 }
 
-// Pd[r][c] = P16[r][c] duplicated into both halves (the B operand of the packed product)
+// Pd[r][c] = P16[r][c] duplicated into both halves (the B operand of the packed product); 128 x Np
 __global__ void k_dup16(const uint16_t *__restrict__ P16, int32_t Np, uint32_t *__restrict__ Pd) {
   const int64_t total = (int64_t)TILE * (Np / 4);
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
@@ -531,7 +619,6 @@ __global__ void k_dup16(const uint16_t *__restrict__ P16, int32_t Np, uint32_t *
   }
 }
 
-// ---- 16-bit row-block sharding (fw_sharded16 below)
 // rows x cols block of int32 (ld lds) -> capped u16 (ld ld16); cols % 4 == 0
 __global__ void k_to16r(const int32_t *__restrict__ S, int64_t lds, uint16_t *__restrict__ S16, int64_t ld16,
                         int64_t rows, int32_t cols) {
@@ -559,21 +646,8 @@ __global__ void k_from16r(const uint16_t *__restrict__ S16, int64_t ld16, int32_
   }
 }
 
-// the assembled int32 pivot row block -> its capped u16 copy and (Pd non-null) the duplicated u32 copy;
-// n = TILE * Np, n % 4 == 0
-__global__ void k_prow_to16(const int32_t *__restrict__ P32, uint16_t *__restrict__ P16, uint32_t *__restrict__ Pd,
-                            int64_t n) {
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n / 4; i += (int64_t)gridDim.x * blockDim.x) {
-    const int4 v = reinterpret_cast<const int4 *>(P32)[i];
-    const uint32_t a = (uint32_t)min(v.x, (int32_t)C16), b = (uint32_t)min(v.y, (int32_t)C16);
-    const uint32_t c = (uint32_t)min(v.z, (int32_t)C16), d = (uint32_t)min(v.w, (int32_t)C16);
-    reinterpret_cast<uint2 *>(P16)[i] = make_uint2(a | (b << 16), c | (d << 16));
-    if (Pd) reinterpret_cast<uint4 *>(Pd)[i] = make_uint4(a * 0x10001u, b * 0x10001u, c * 0x10001u, d * 0x10001u);
-  }
-}
-
 // k_check16 over a rank's owned UPPER tiles (the authoritative ones; D is symmetric, so the ranks
-// together cover every pair): a capped entry of a connected pair sets *flag = -1 (MIN-reducible)
+// together cover every pair): a capped entry of a connected pair sets *flag = -1
 __global__ void k_check16_list(const uint16_t *__restrict__ S16, int64_t ld16, const int32_t *__restrict__ orow,
                                int32_t nown, int32_t Np, const int32_t *__restrict__ lab, int32_t n_real,
                                int32_t *flag) {
@@ -598,497 +672,150 @@ __global__ void k_check16_list(const uint16_t *__restrict__ S16, int64_t ld16, c
   if (__syncthreads_or(found) && threadIdx.x == 0) atomicMin(flag, -1);
 }
 
-// Closure of the 16-bit pivot tile (ld ldt) in place, packed like the tile kernel: thread (ty, tx)
-// owns rows {ty*4 .. +3, 64 + ty*4 .. +3} as 4 row PAIRS and columns {tx*4 .. +3, 64 + tx*4 .. +3},
-// c[p][q] = (T[i][j], T[i+1][j]); step kk reads row kk from shared memory -- it is also column kk, the
-// tile being symmetric -- as the row-pair operand and, duplicated, as the column operand, so one
-// VIADDMNMX.U16x2 relaxes two entries (values <= C16: sums <= 0xFFFE never wrap, results stay
-// <= C16).  About 60 registers: it fits beside two CTAs of the tile kernel, which the lookahead
-// needs (the int32-register closure took 108 x 256 registers, more than an SM has left then, so it
-// waited for every rest-of-round launch to drain).
-__global__ void __launch_bounds__(NT, 1) k_fw_phase1_16(uint16_t *T, int64_t ldt) {
-  __shared__ __align__(16) uint16_t rowbuf[2][TILE];
-  const int tx = threadIdx.x & 15, ty = threadIdx.x >> 4;
-  uint32_t c[4][8];
-#pragma unroll
-  for (int p = 0; p < 4; ++p) {
-    const int i = (p < 2 ? 0 : 64) + ty * 4 + (p & 1) * 2;
-#pragma unroll
-    for (int h = 0; h < 2; ++h) {
-      const uint2 v = *reinterpret_cast<const uint2 *>(T + (int64_t)i * ldt + h * 64 + tx * 4);
-      const uint2 w = *reinterpret_cast<const uint2 *>(T + (int64_t)(i + 1) * ldt + h * 64 + tx * 4);
-      c[p][h * 4 + 0] = __byte_perm(v.x, w.x, 0x5410);
-      c[p][h * 4 + 1] = __byte_perm(v.x, w.x, 0x7632);
-      c[p][h * 4 + 2] = __byte_perm(v.y, w.y, 0x5410);
-      c[p][h * 4 + 3] = __byte_perm(v.y, w.y, 0x7632);
+// ------------------------------------------------------------------------------ sharding kernels
+// Pivot-row block <-> a rank's owned storage, round k (L: 128 x Np, leading dimension Np).
+//   dir = 0 (gather):  L[:, ti-block] = S(ti, k)^T for owned ti < k; L[:, j >= k] = S(k, j) if row k owned
+//   dir = 1 (scatter): the inverse, from the completed (phase-2-updated) block
+// Grid (16 sub-blocks of 32 x 32, npieces), 256 threads: pieces [0, nrow) are the tiles j = k + y of the
+// pivot row when this rank owns it (nrow = nt - k, local row posk), the next mk the owned rows ti < k.
+template <class E>
+__global__ void k_prow_xfer(E *S, int64_t ldd, const int32_t *orow, int32_t k, int32_t nt, int32_t posk, E *L,
+                            int32_t Np, int dir) {
+  __shared__ E t[32][33];
+  const int nrow = posk >= 0 ? nt - k : 0;
+  const int y = blockIdx.y;
+  const int bx = blockIdx.x & 3, by = blockIdx.x >> 2;         // 32 x 32 sub-block (bx: x, by: y)
+  const int lx = threadIdx.x & 31, ly = threadIdx.x >> 5;      // 32 x 8 threads
+  if (y < nrow) {              // the pivot row's upper part: plain copy, tiles j >= k
+    const int lr = posk, tj = k + y;
+    for (int yy = ly; yy < 32; yy += 8) {
+      const int64_t row = by * 32 + yy, col = (int64_t)tj * TILE + bx * 32 + lx;
+      E *sp = S + ((int64_t)lr * TILE + row) * ldd + col;
+      E *pp = L + row * Np + col;
+      if (dir == 0) *pp = *sp; else *sp = *pp;
     }
+    return;
   }
-  if (threadIdx.x < TILE / 4)   // row 0
-    reinterpret_cast<uint2 *>(rowbuf[0])[threadIdx.x] = reinterpret_cast<const uint2 *>(T)[threadIdx.x];
-  __syncthreads();
-  for (int kk = 0; kk < TILE; ++kk) {
-    const uint16_t *rb = rowbuf[kk & 1];
-    const uint2 alo = *reinterpret_cast<const uint2 *>(rb + ty * 4);        // rows ty*4 .. +3 (pairs)
-    const uint2 ahi = *reinterpret_cast<const uint2 *>(rb + 64 + ty * 4);
-    const uint2 blo = *reinterpret_cast<const uint2 *>(rb + tx * 4);        // columns tx*4 .. +3
-    const uint2 bhi = *reinterpret_cast<const uint2 *>(rb + 64 + tx * 4);
-    const uint32_t a[4] = {alo.x, alo.y, ahi.x, ahi.y};
-    const uint32_t b[8] = {__byte_perm(blo.x, 0, 0x1010), __byte_perm(blo.x, 0, 0x3232),
-                           __byte_perm(blo.y, 0, 0x1010), __byte_perm(blo.y, 0, 0x3232),
-                           __byte_perm(bhi.x, 0, 0x1010), __byte_perm(bhi.x, 0, 0x3232),
-                           __byte_perm(bhi.y, 0, 0x1010), __byte_perm(bhi.y, 0, 0x3232)};
-#pragma unroll
-    for (int p = 0; p < 4; ++p)
-#pragma unroll
-      for (int q = 0; q < 8; ++q) c[p][q] = __viaddmin_u16x2(a[p], b[q], c[p][q]);
-    const int nk = kk + 1;   // its owner publishes row nk for the next step
-    if (nk < TILE && ty == ((nk & 63) >> 2)) {
-      const int p = ((nk & 3) >> 1) + (nk >= 64 ? 2 : 0), hi = nk & 1;
-      uint16_t *wb = rowbuf[nk & 1];
-#pragma unroll
-      for (int pp = 0; pp < 4; ++pp) {
-        if (pp == p) {
-          const uint32_t sel = hi ? 0x7632 : 0x5410;
-          *reinterpret_cast<uint2 *>(wb + tx * 4) =
-              make_uint2(__byte_perm(c[pp][0], c[pp][1], sel), __byte_perm(c[pp][2], c[pp][3], sel));
-          *reinterpret_cast<uint2 *>(wb + 64 + tx * 4) =
-              make_uint2(__byte_perm(c[pp][4], c[pp][5], sel), __byte_perm(c[pp][6], c[pp][7], sel));
-        }
-      }
-    }
+  const int lr = y - nrow, ti = orow[lr];   // owned row below the pivot: tile (ti, k) <-> L[:, ti-block]^T
+  if (dir == 0) {
+    for (int yy = ly; yy < 32; yy += 8)   // S rows ti-block (bx*32+yy), cols k-block (by*32+lx)
+      t[yy][lx] = S[((int64_t)lr * TILE + bx * 32 + yy) * ldd + (int64_t)k * TILE + by * 32 + lx];
     __syncthreads();
-  }
-#pragma unroll
-  for (int p = 0; p < 4; ++p) {
-    const int i = (p < 2 ? 0 : 64) + ty * 4 + (p & 1) * 2;
-#pragma unroll
-    for (int h = 0; h < 2; ++h) {
-      const uint32_t *cc = &c[p][h * 4];
-      *reinterpret_cast<uint2 *>(T + (int64_t)i * ldt + h * 64 + tx * 4) =
-          make_uint2(__byte_perm(cc[0], cc[1], 0x5410), __byte_perm(cc[2], cc[3], 0x5410));
-      *reinterpret_cast<uint2 *>(T + (int64_t)(i + 1) * ldt + h * 64 + tx * 4) =
-          make_uint2(__byte_perm(cc[0], cc[1], 0x7632), __byte_perm(cc[2], cc[3], 0x7632));
-    }
-  }
-}
-
-// Phases 2 and 3, packed: the same persistent TMA-ring structure as k_fw_tiles.  A^T chunks are 16-bit
-// rows of the pivot row block (tmA: KC x 128 u16), B chunks rows of its duplicated copy Pd (tmB: KC x
-// 128 u32).  Thread (ty, tx) owns rows {ty*4 .. +3, 64 + ty*4 .. +3} as 4 row PAIRS and columns
-// {tx*4 .. +3, 64 + tx*4 .. +3}: c[r2][q] = (C[i][j], C[i+1][j]) packed, so one VIADDMNMX.U16x2
-// c = min(c, a_pair + b_dup) does two min-plus.
-struct TileJob16 {
-  uint16_t *C;       // matrix holding the C tiles, leading dimension ldc (u16 elements)
-  int64_t ldc;
-  int32_t a_row0;    // row of the pivot row block inside tmA
-  int32_t k, nt;
-  int32_t mode;      // MODE_PIVOT_ROW, MODE_UPPER, MODE_CROSS, MODE_REST or MODE_LIST
-  int32_t mirror;
-  int64_t ntiles;
-  // MODE_LIST (row-block sharded): as TileJob -- C holds the rank's owned tile rows only
-  const int32_t *orow;
-  const int64_t *opre;
-  int32_t nown, mk, posk;
-  unsigned long long *dbg;   // development (EAR_FW16_DBG): per-CTA %globaltimer at start / end, or null
-  int32_t ti0;               // first tile row held by C (MODE_PIVOT_ROW on a standalone pivot row block: k)
-  int32_t posk1;             // MODE_LIST_CROSS / _REST
-  int32_t *counter;          // kDYN: {next tile, CTAs done}, zero at launch, reset by the last CTA
-};
-
-// LAR = 1: a ring stage is refilled by the LAST warp to finish consuming it (a shared counter) instead
-// of thread 0 waiting on an 'empty' barrier at the start of each chunk (which ties warp 0 to the
-// slowest warp every chunk).
-template <int KC, int STAGES, int MINB, int UNR, int NTH = 256, int PFC = 0, int LAR = 0, int SPIN = 0,
-          int DYN = 0, int HINT = 0>
-struct Fw16Cfg {
-  static constexpr int NCHUNK = TILE / KC;
-  static constexpr int A_CHUNK = KC * TILE;   // u16 elements
-  static constexpr int B_CHUNK = KC * TILE;   // u32 elements
-  static constexpr int SMEM = STAGES * (A_CHUNK * 2 + B_CHUNK * 4) + 2 * STAGES * 8 + STAGES * 4 + 8;
-  static constexpr int kKC = KC, kSTAGES = STAGES, kMINB = MINB, kUNR = UNR, kNTH = NTH, kPFC = PFC, kLAR = LAR;
-  static constexpr int kSPIN = SPIN, kDYN = DYN, kHINT = HINT;
-  static constexpr int RPH = 256 * 2 / NTH;   // row pairs per 64-row half owned by a thread (2 or 4)
-};
-
-__device__ __forceinline__ void decode16(const TileJob16 &J, int64_t idx, int &ti, int &tj, int &lr) {
-  TileJob T{};
-  T.k = J.k; T.nt = J.nt; T.mode = J.mode; T.ti0 = J.ti0;
-  T.orow = J.orow; T.opre = J.opre; T.nown = J.nown; T.mk = J.mk; T.posk = J.posk; T.posk1 = J.posk1;
-  decode_tile(T, idx, ti, tj, lr);
-}
-
-// Thread (ty, tx): columns {tx*4 .. +3, 64 + tx*4 .. +3}; rows {h*64 + ty*2*RPH + 2p, +1} for h = 0, 1 and
-// p < RPH, i.e. 2*RPH row pairs (8 with 256 threads, 16 with 128).
-template <class CF>
-__global__ void __launch_bounds__(CF::kNTH, CF::kMINB)
-    k_fw_tiles16(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB, const TileJob16 J) {
-  constexpr int KC = CF::kKC, NCHUNK = CF::NCHUNK, STAGES = CF::kSTAGES, NTH = CF::kNTH, RPH = CF::RPH;
-  constexpr int NRP = 2 * RPH;   // row pairs per thread
-  extern __shared__ __align__(128) uint8_t smem16[];
-  uint16_t *sA = reinterpret_cast<uint16_t *>(smem16);                        // [STAGES][KC][TILE] u16
-  uint32_t *sB = reinterpret_cast<uint32_t *>(sA + STAGES * CF::A_CHUNK);     // [STAGES][KC][TILE] u32
-  uint64_t *full = reinterpret_cast<uint64_t *>(sB + STAGES * CF::B_CHUNK);
-  uint64_t *empty = full + STAGES;
-  int32_t *cnt = reinterpret_cast<int32_t *>(empty + STAGES);   // LAR: warps done with the stage
-  const int tid = threadIdx.x, lane = tid & 31;
-  const int tx = tid & 15, ty = tid >> 4;
-  if (J.dbg && tid == 0) {
-    unsigned long long t;
-    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
-    uint32_t smid;
-    asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
-    J.dbg[3 * blockIdx.x] = t;
-    J.dbg[3 * blockIdx.x + 2] = smid;
-  }
-
-  const int my_tiles = J.ntiles > (int64_t)blockIdx.x ? (int)((J.ntiles - 1 - blockIdx.x) / gridDim.x + 1) : 0;
-  const int total_chunks = my_tiles * NCHUNK;
-  int issued = 0;
-  auto tile_of = [&](int it, int &ti, int &tj, int &lr) { decode16(J, blockIdx.x + (int64_t)it * gridDim.x, ti, tj, lr); };
-  auto issue = [&](int c, int st) {   // chunk c into stage st
-    int pti, ptj, plr;
-    tile_of(c / NCHUNK, pti, ptj, plr);
-    const int kc = c % NCHUNK;
-    mbar_arrive_tx(&full[st], CF::A_CHUNK * 2 + CF::B_CHUNK * 4);
-    tma_load_2d(sA + st * CF::A_CHUNK, &tmA, pti * TILE, J.a_row0 + kc * KC, &full[st]);
-    tma_load_2d(sB + st * CF::B_CHUNK, &tmB, ptj * TILE, kc * KC, &full[st]);
-  };
-  auto produce = [&](int upto) {
-    while (issued < upto) {
-      const int st = issued % STAGES;
-      if (issued >= STAGES) mbar_wait(&empty[st], (uint32_t)((issued / STAGES - 1) & 1));
-      int pti, ptj, plr;
-      tile_of(issued / NCHUNK, pti, ptj, plr);
-      const int kc = issued % NCHUNK;
-      mbar_arrive_tx(&full[st], CF::A_CHUNK * 2 + CF::B_CHUNK * 4);
-      tma_load_2d(sA + st * CF::A_CHUNK, &tmA, pti * TILE, J.a_row0 + kc * KC, &full[st]);
-      tma_load_2d(sB + st * CF::B_CHUNK, &tmB, ptj * TILE, kc * KC, &full[st]);
-      ++issued;
-    }
-  };
-  if (tid == 0) {
-    for (int s = 0; s < STAGES; ++s) {
-      mbar_init(&full[s], 1);
-      mbar_init(&empty[s], NTH / 32);
-      cnt[s] = 0;
-    }
-    asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
-    asm volatile("prefetch.tensormap [%0];\n" ::"l"(reinterpret_cast<uint64_t>(&tmA)) : "memory");
-    asm volatile("prefetch.tensormap [%0];\n" ::"l"(reinterpret_cast<uint64_t>(&tmB)) : "memory");
-  }
-  __syncthreads();
-  if (tid == 0 && my_tiles > 0) {
-    if (CF::kLAR) {
-      for (int c = 0; c < STAGES && c < total_chunks; ++c) issue(c, c);
-    } else {
-      produce(total_chunks < STAGES ? total_chunks : STAGES);
-    }
-  }
-
-  auto row_of = [&](int r2) { return (r2 < RPH ? 0 : 64) + ty * 2 * RPH + (r2 % RPH) * 2; };
-  int g = 0;
-  for (int it = 0; it < my_tiles; ++it) {
-    int ti, tj, lr;
-    tile_of(it, ti, tj, lr);
-    uint32_t c[NRP][8];
-    uint16_t *Ct = J.C + (int64_t)lr * TILE * J.ldc + (int64_t)tj * TILE;
-#pragma unroll
-    for (int r2 = 0; r2 < NRP; ++r2) {
-      const int i = row_of(r2);
-#pragma unroll
-      for (int h = 0; h < 2; ++h) {
-        const uint2 v = *reinterpret_cast<const uint2 *>(Ct + (int64_t)i * J.ldc + h * 64 + tx * 4);
-        const uint2 w = *reinterpret_cast<const uint2 *>(Ct + (int64_t)(i + 1) * J.ldc + h * 64 + tx * 4);
-        c[r2][h * 4 + 0] = __byte_perm(v.x, w.x, 0x5410);
-        c[r2][h * 4 + 1] = __byte_perm(v.x, w.x, 0x7632);
-        c[r2][h * 4 + 2] = __byte_perm(v.y, w.y, 0x5410);
-        c[r2][h * 4 + 3] = __byte_perm(v.y, w.y, 0x7632);
-      }
-    }
-    if (CF::kPFC && it + 1 < my_tiles) {   // pull the next tile's C rows into L2 while this one computes
-      int nti, ntj, nlr;
-      tile_of(it + 1, nti, ntj, nlr);
-      const uint16_t *Cn = J.C + (int64_t)nlr * TILE * J.ldc + (int64_t)ntj * TILE;
-      // 128 rows x 256 B: one 128-byte line per (row, half), spread over the CTA's threads
-      for (int l = tid; l < 2 * TILE; l += NTH)
-        asm volatile("prefetch.global.L2::evict_last [%0];" ::"l"(Cn + (int64_t)(l >> 1) * J.ldc + (l & 1) * 64));
-    }
-#pragma unroll 1
-    for (int kc = 0; kc < NCHUNK; ++kc, ++g) {
-      if (!CF::kLAR && tid == 0) produce(g + STAGES < total_chunks ? g + STAGES : total_chunks);
-      const int st = g % STAGES;
-      if (CF::kSPIN) mbar_wait_spin(&full[st], (uint32_t)((g / STAGES) & 1));
-      else mbar_wait(&full[st], (uint32_t)((g / STAGES) & 1));
-      const uint16_t *a_s = sA + st * CF::A_CHUNK;
-      const uint32_t *b_s = sB + st * CF::B_CHUNK;
-#pragma unroll CF::kUNR
-      for (int kk = 0; kk < KC; ++kk) {
-        uint32_t a[NRP];
-        if (RPH == 2) {
-          const uint2 alo = *reinterpret_cast<const uint2 *>(a_s + kk * TILE + ty * 4);
-          const uint2 ahi = *reinterpret_cast<const uint2 *>(a_s + kk * TILE + 64 + ty * 4);
-          a[0] = alo.x; a[1] = alo.y; a[RPH] = ahi.x; a[RPH + 1] = ahi.y;
-        } else {
-          const uint4 alo = *reinterpret_cast<const uint4 *>(a_s + kk * TILE + ty * 8);
-          const uint4 ahi = *reinterpret_cast<const uint4 *>(a_s + kk * TILE + 64 + ty * 8);
-          a[0] = alo.x; a[1] = alo.y; a[2] = alo.z; a[3] = alo.w;
-          a[RPH] = ahi.x; a[RPH + 1] = ahi.y; a[RPH + 2] = ahi.z; a[RPH + 3] = ahi.w;
-        }
-        const uint4 blo = *reinterpret_cast<const uint4 *>(b_s + kk * TILE + tx * 4);
-        const uint4 bhi = *reinterpret_cast<const uint4 *>(b_s + kk * TILE + 64 + tx * 4);
-        const uint32_t b[8] = {blo.x, blo.y, blo.z, blo.w, bhi.x, bhi.y, bhi.z, bhi.w};
-#pragma unroll
-        for (int r2 = 0; r2 < NRP; ++r2)
-#pragma unroll
-          for (int q = 0; q < 8; ++q) c[r2][q] = __viaddmin_u16x2(a[r2], b[q], c[r2][q]);
-      }
-      __syncwarp();
-      if (CF::kLAR) {
-        if (lane == 0) {
-          __threadfence_block();
-          if (atomicAdd(&cnt[st], 1) == NTH / 32 - 1) {   // the last reader of this stage refills it
-            cnt[st] = 0;
-            __threadfence_block();
-            asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");
-            if (g + STAGES < total_chunks) issue(g + STAGES, st);
-          }
-        }
-      } else if (lane == 0) {
-        mbar_arrive(&empty[st]);
-      }
-    }
-#pragma unroll
-    for (int r2 = 0; r2 < NRP; ++r2) {
-      const int i = row_of(r2);
-#pragma unroll
-      for (int h = 0; h < 2; ++h) {
-        const uint32_t *cc = &c[r2][h * 4];
-        *reinterpret_cast<uint2 *>(Ct + (int64_t)i * J.ldc + h * 64 + tx * 4) =
-            make_uint2(__byte_perm(cc[0], cc[1], 0x5410), __byte_perm(cc[2], cc[3], 0x5410));
-        *reinterpret_cast<uint2 *>(Ct + (int64_t)(i + 1) * J.ldc + h * 64 + tx * 4) =
-            make_uint2(__byte_perm(cc[0], cc[1], 0x7632), __byte_perm(cc[2], cc[3], 0x7632));
-      }
-    }
-    if (J.mirror && ti != tj) {
-      uint16_t *Mt = J.C + (int64_t)tj * TILE * J.ldc + (int64_t)ti * TILE;
-#pragma unroll
-      for (int q = 0; q < 8; ++q) {
-        const int j = (q < 4 ? 0 : 64) + tx * 4 + (q & 3);
-#pragma unroll
-        for (int h = 0; h < 2; ++h) {
-          if (RPH == 2) {
-            *reinterpret_cast<uint2 *>(Mt + (int64_t)j * J.ldc + h * 64 + ty * 4) = make_uint2(c[h * 2][q], c[h * 2 + 1][q]);
-          } else {
-            *reinterpret_cast<uint4 *>(Mt + (int64_t)j * J.ldc + h * 64 + ty * 8) =
-                make_uint4(c[h * 4][q], c[h * 4 + 1][q], c[h * 4 + 2][q], c[h * 4 + 3][q]);
-          }
-        }
-      }
-    }
-  }
-  if (J.dbg) {
+    for (int yy = ly; yy < 32; yy += 8)   // L rows (by*32+yy), cols ti-block (bx*32+lx)
+      L[(int64_t)(by * 32 + yy) * Np + (int64_t)ti * TILE + bx * 32 + lx] = t[lx][yy];
+  } else {
+    for (int yy = ly; yy < 32; yy += 8)
+      t[yy][lx] = L[(int64_t)(by * 32 + yy) * Np + (int64_t)ti * TILE + bx * 32 + lx];
     __syncthreads();
-    if (tid == 0) {
-      unsigned long long t;
-      asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
-      J.dbg[3 * blockIdx.x + 1] = t;
+    for (int yy = ly; yy < 32; yy += 8)
+      S[((int64_t)lr * TILE + bx * 32 + yy) * ldd + (int64_t)k * TILE + by * 32 + lx] = t[lx][yy];
+  }
+}
+
+// The per-round broadcast of the pieces: this rank's column blocks of the phase-2-updated pivot row
+// block (k .. nt-1 when it owns row k, then its owned rows below k -- see k_prow_xfer) are copied from
+// L into the same positions of every destination block dst.p[d] (the peers' stage buffers, mapped over
+// NVLink, and its own).  Grid (max(npieces, 1), 4 row quarters).  With `counter` the last CTA to finish
+// raises flag slot `slot` of every window in `flags` to `value` (system-scope release after every CTA's
+// stores are fenced: a peer that sees the flag sees the data).
+template <class E>
+__global__ void k_push_pieces(const E *__restrict__ L, int32_t Np, int32_t k, int32_t nt, int32_t posk, int32_t mk,
+                              const int32_t *__restrict__ orow, PeerPtrs dst, int32_t *counter, PeerPtrs flags,
+                              int32_t slot, uint64_t value) {
+  const int nrow = posk >= 0 ? nt - k : 0;
+  const int y = blockIdx.x;
+  if (y < nrow + mk) {
+    const int cb = y < nrow ? k + y : orow[y - nrow];
+    constexpr int V = 16 / (int)sizeof(E);   // elements per 16-byte vector
+    constexpr int PER_ROW = TILE / V;
+    for (int i = threadIdx.x; i < 32 * PER_ROW; i += blockDim.x) {
+      const int r = blockIdx.y * 32 + i / PER_ROW, c = (i % PER_ROW) * V;
+      const int64_t off = (int64_t)r * Np + (int64_t)cb * TILE + c;
+      const uint4 v = *reinterpret_cast<const uint4 *>(L + off);
+      for (int d = 0; d < dst.n; ++d) *reinterpret_cast<uint4 *>(reinterpret_cast<E *>(dst.p[d]) + off) = v;
+    }
+  }
+  if (!counter) return;
+  __threadfence_system();
+  __syncthreads();
+  if (threadIdx.x == 0 && atomicAdd(counter, 1) == (int)(gridDim.x * gridDim.y) - 1) {
+    *counter = 0;   // the next push on this stream starts from zero
+    __threadfence_system();
+    for (int d = 0; d < flags.n; ++d) {
+      uint64_t *f = reinterpret_cast<uint64_t *>(flags.p[d]) + slot;
+      asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(f), "l"(value) : "memory");
     }
   }
 }
 
-// Dynamically scheduled version of k_fw_tiles16 (CF::kDYN): a CTA takes its next tile from a global
-// counter when it issues that tile's first TMA chunk, instead of the static blockIdx + it * grid
-// assignment.  Measured with the static assignment (tools/fw16_cta_times.py): all CTAs start
-// together but end between 43 % and 100 % of the launch -- the SM's warp scheduler favours its oldest
-// CTA, so the three CTAs of an SM run at different speeds and each SM spends the last part of every
-// launch with one or two of them (2.15 resident CTAs on average).  With the counter, fast CTAs simply
-// take more tiles.  The tile of a CTA's tile sequence number q is published in tslot[q & 1] (tagged
-// with q) by the thread that issues its first chunk; the ring depth (2) never exceeds the chunks per
-// tile (4), so a slot is rewritten only after every warp has read it.  The last CTA to finish resets
-// the counter pair for the next launch on the same stream.
-template <class CF>
-__global__ void __launch_bounds__(CF::kNTH, CF::kMINB)
-    k_fw_tiles16_dyn(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
-                     const TileJob16 J) {
-  constexpr int KC = CF::kKC, NCHUNK = CF::NCHUNK, STAGES = CF::kSTAGES, NTH = CF::kNTH, RPH = CF::RPH;
-  constexpr int NRP = 2 * RPH, NW = NTH / 32;
-  static_assert(NCHUNK >= STAGES, "tile slots are rewritten only after every warp has read them");
-  constexpr int32_t NONE = 0xFFFFF;
-  extern __shared__ __align__(128) uint8_t smem16[];
-  uint16_t *sA = reinterpret_cast<uint16_t *>(smem16);
-  uint32_t *sB = reinterpret_cast<uint32_t *>(sA + STAGES * CF::A_CHUNK);
-  uint64_t *full = reinterpret_cast<uint64_t *>(sB + STAGES * CF::B_CHUNK);
-  int32_t *cnt = reinterpret_cast<int32_t *>(full + 2 * STAGES);   // [STAGES] warps done with the stage
-  int32_t *tslot = cnt + STAGES;                                   // [2] (q << 20) | tile
-  const int tid = threadIdx.x, lane = tid & 31;
-  const int tx = tid & 15, ty = tid >> 4;
-  if (J.dbg && tid == 0) {
-    unsigned long long t;
-    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
-    uint32_t smid;
-    asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
-    J.dbg[3 * blockIdx.x] = t;
-    J.dbg[3 * blockIdx.x + 2] = smid;
+// the range-check bit of this rank -> CHECK slot `slot` of every window, value (seq << 1) | bad
+__global__ void k_check_push(const int32_t *flag, PeerPtrs wins, int32_t slot, uint64_t seq) {
+  const uint64_t v = (seq << 1) | (uint64_t)(*flag < 0 ? 1 : 0);
+  __threadfence_system();
+  for (int d = threadIdx.x; d < wins.n; d += blockDim.x) {
+    uint64_t *f = reinterpret_cast<uint64_t *>(wins.p[d]) + slot;
+    asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(f), "l"(v) : "memory");
   }
-  // chunk c of this CTA's sequence into stage st (one thread)
-  auto issue = [&](int c, int st) {
-    const int q = c / NCHUNK, kc = c % NCHUNK;
-    int32_t t;
-    if (kc == 0) {
-      const int32_t tt = atomicAdd(J.counter, 1);
-      t = tt < J.ntiles ? tt : -1;
-      tslot[q & 1] = (q << 20) | (t < 0 ? NONE : t);
-      __threadfence_block();
-    } else {
-      const int32_t v = tslot[q & 1] & NONE;
-      t = v == NONE ? -1 : v;
+}
+// OR of the ranks' bits (this rank's window, slots [slot, slot + P)) -> *flag = -1 if any is set
+__global__ void k_check_fold(const uint64_t *slots, int32_t P, int32_t *flag) {
+  if (threadIdx.x == 0) {
+    int any = 0;
+    for (int p = 0; p < P; ++p) {
+      uint64_t v;
+      asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(slots + p) : "memory");
+      any |= (int)(v & 1);
     }
-    if (t < 0) {   // no tile: complete the phase without data so that the waiters see the end
-      mbar_arrive(&full[st]);
-      return;
-    }
-    int pti, ptj, plr;
-    decode16(J, t, pti, ptj, plr);
-    mbar_arrive_tx(&full[st], CF::A_CHUNK * 2 + CF::B_CHUNK * 4);
-    if (CF::kHINT) {   // the pivot row block stays in L2 while the C tiles stream through it
-      uint64_t pol;
-      asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
-      tma_load_2d_hint(sA + st * CF::A_CHUNK, &tmA, pti * TILE, J.a_row0 + kc * KC, &full[st], pol);
-      tma_load_2d_hint(sB + st * CF::B_CHUNK, &tmB, ptj * TILE, kc * KC, &full[st], pol);
-    } else {
-      tma_load_2d(sA + st * CF::A_CHUNK, &tmA, pti * TILE, J.a_row0 + kc * KC, &full[st]);
-      tma_load_2d(sB + st * CF::B_CHUNK, &tmB, ptj * TILE, kc * KC, &full[st]);
-    }
-  };
-  if (tid == 0) {
-    for (int s = 0; s < STAGES; ++s) {
-      mbar_init(&full[s], 1);
-      cnt[s] = 0;
-    }
-    asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
-    asm volatile("prefetch.tensormap [%0];\n" ::"l"(reinterpret_cast<uint64_t>(&tmA)) : "memory");
-    asm volatile("prefetch.tensormap [%0];\n" ::"l"(reinterpret_cast<uint64_t>(&tmB)) : "memory");
+    *flag = any ? -1 : 0;
   }
-  __syncthreads();
-  if (tid == 0)
-    for (int c = 0; c < STAGES; ++c) issue(c, c);
+}
 
-  auto row_of = [&](int r2) { return (r2 < RPH ? 0 : 64) + ty * 2 * RPH + (r2 % RPH) * 2; };
-  int g = 0;
-  for (int q = 0;; ++q) {
-    mbar_wait(&full[g % STAGES], (uint32_t)((g / STAGES) & 1));
-    const int32_t v = tslot[q & 1] & NONE;
-    if (v == NONE) break;
-    int ti, tj, lr;
-    decode16(J, v, ti, tj, lr);
-    uint32_t c[NRP][8];
-    uint16_t *Ct = J.C + (int64_t)lr * TILE * J.ldc + (int64_t)tj * TILE;
-#pragma unroll
-    for (int r2 = 0; r2 < NRP; ++r2) {
-      const int i = row_of(r2);
-#pragma unroll
-      for (int h = 0; h < 2; ++h) {
-        const uint2 *pa = reinterpret_cast<const uint2 *>(Ct + (int64_t)i * J.ldc + h * 64 + tx * 4);
-        const uint2 *pb = reinterpret_cast<const uint2 *>(Ct + (int64_t)(i + 1) * J.ldc + h * 64 + tx * 4);
-        const uint2 a = CF::kHINT ? __ldcs(pa) : *pa;
-        const uint2 b = CF::kHINT ? __ldcs(pb) : *pb;
-        c[r2][h * 4 + 0] = __byte_perm(a.x, b.x, 0x5410);
-        c[r2][h * 4 + 1] = __byte_perm(a.x, b.x, 0x7632);
-        c[r2][h * 4 + 2] = __byte_perm(a.y, b.y, 0x5410);
-        c[r2][h * 4 + 3] = __byte_perm(a.y, b.y, 0x7632);
-      }
-    }
-#pragma unroll 1
-    for (int kc = 0; kc < NCHUNK; ++kc, ++g) {
-      const int st = g % STAGES;
-      if (kc > 0) mbar_wait(&full[st], (uint32_t)((g / STAGES) & 1));
-      if (CF::kPFC && kc == NCHUNK - 1) {   // the next tile, once published: its C rows into L2
-        const int32_t nv = tslot[(q + 1) & 1];
-        if ((nv >> 20) == q + 1 && (nv & NONE) != NONE) {
-          int nti, ntj, nlr;
-          decode16(J, nv & NONE, nti, ntj, nlr);
-          const uint16_t *Cn = J.C + (int64_t)nlr * TILE * J.ldc + (int64_t)ntj * TILE;
-          for (int l = tid; l < 2 * TILE; l += NTH)
-            asm volatile("prefetch.global.L2::evict_last [%0];" ::"l"(Cn + (int64_t)(l >> 1) * J.ldc + (l & 1) * 64));
-        }
-      }
-      const uint16_t *a_s = sA + st * CF::A_CHUNK;
-      const uint32_t *b_s = sB + st * CF::B_CHUNK;
-#pragma unroll CF::kUNR
-      for (int kk = 0; kk < KC; ++kk) {
-        uint32_t a[NRP];
-        if (RPH == 2) {
-          const uint2 alo = *reinterpret_cast<const uint2 *>(a_s + kk * TILE + ty * 4);
-          const uint2 ahi = *reinterpret_cast<const uint2 *>(a_s + kk * TILE + 64 + ty * 4);
-          a[0] = alo.x; a[1] = alo.y; a[RPH] = ahi.x; a[RPH + 1] = ahi.y;
-        } else {
-          const uint4 alo = *reinterpret_cast<const uint4 *>(a_s + kk * TILE + ty * 8);
-          const uint4 ahi = *reinterpret_cast<const uint4 *>(a_s + kk * TILE + 64 + ty * 8);
-          a[0] = alo.x; a[1] = alo.y; a[2] = alo.z; a[3] = alo.w;
-          a[RPH] = ahi.x; a[RPH + 1] = ahi.y; a[RPH + 2] = ahi.z; a[RPH + 3] = ahi.w;
-        }
-        const uint4 blo = *reinterpret_cast<const uint4 *>(b_s + kk * TILE + tx * 4);
-        const uint4 bhi = *reinterpret_cast<const uint4 *>(b_s + kk * TILE + 64 + tx * 4);
-        const uint32_t b[8] = {blo.x, blo.y, blo.z, blo.w, bhi.x, bhi.y, bhi.z, bhi.w};
-#pragma unroll
-        for (int r2 = 0; r2 < NRP; ++r2)
-#pragma unroll
-          for (int qq = 0; qq < 8; ++qq) c[r2][qq] = __viaddmin_u16x2(a[r2], b[qq], c[r2][qq]);
-      }
-      __syncwarp();
-      if (lane == 0) {
-        __threadfence_block();
-        if (atomicAdd(&cnt[st], 1) == NW - 1) {   // the last reader of this stage refills it
-          cnt[st] = 0;
-          __threadfence_block();
-          asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");
-          issue(g + STAGES, st);
-        }
-      }
-    }
-#pragma unroll
-    for (int r2 = 0; r2 < NRP; ++r2) {
-      const int i = row_of(r2);
-#pragma unroll
-      for (int h = 0; h < 2; ++h) {
-        const uint32_t *cc = &c[r2][h * 4];
-        uint2 *qa = reinterpret_cast<uint2 *>(Ct + (int64_t)i * J.ldc + h * 64 + tx * 4);
-        uint2 *qb = reinterpret_cast<uint2 *>(Ct + (int64_t)(i + 1) * J.ldc + h * 64 + tx * 4);
-        const uint2 va = make_uint2(__byte_perm(cc[0], cc[1], 0x5410), __byte_perm(cc[2], cc[3], 0x5410));
-        const uint2 vb = make_uint2(__byte_perm(cc[0], cc[1], 0x7632), __byte_perm(cc[2], cc[3], 0x7632));
-        if (CF::kHINT) { __stcs(qa, va); __stcs(qb, vb); } else { *qa = va; *qb = vb; }
-      }
-    }
-    if (J.mirror && ti != tj) {
-      uint16_t *Mt = J.C + (int64_t)tj * TILE * J.ldc + (int64_t)ti * TILE;
-#pragma unroll
-      for (int qq = 0; qq < 8; ++qq) {
-        const int j = (qq < 4 ? 0 : 64) + tx * 4 + (qq & 3);
-#pragma unroll
-        for (int h = 0; h < 2; ++h) {
-          if (RPH == 2) {
-            *reinterpret_cast<uint2 *>(Mt + (int64_t)j * J.ldc + h * 64 + ty * 4) = make_uint2(c[h * 2][qq], c[h * 2 + 1][qq]);
-          } else {
-            *reinterpret_cast<uint4 *>(Mt + (int64_t)j * J.ldc + h * 64 + ty * 8) =
-                make_uint4(c[h * 4][qq], c[h * 4 + 1][qq], c[h * 4 + 2][qq], c[h * 4 + 3][qq]);
-          }
-        }
-      }
-    }
+// owned upper tiles (ti, tj >= ti) -> full D, and their transposed mirrors (tj, ti)  (emulated ranks)
+// grid: (16 sub-blocks, nt column tiles, nown owned rows), 256 threads
+__global__ void k_scatter_upper(const int32_t *S, int64_t ldd, const int32_t *orow, int32_t *Df, int64_t ldf) {
+  __shared__ int32_t t[32][33];
+  const int lr = blockIdx.z, ti = orow[lr], tj = blockIdx.y;
+  if (tj < ti) return;
+  const int bx = blockIdx.x & 3, by = blockIdx.x >> 2;
+  const int lx = threadIdx.x & 31, ly = threadIdx.x >> 5;
+  for (int yy = ly; yy < 32; yy += 8) {
+    const int32_t v = S[((int64_t)lr * TILE + by * 32 + yy) * ldd + (int64_t)tj * TILE + bx * 32 + lx];
+    Df[((int64_t)ti * TILE + by * 32 + yy) * ldf + (int64_t)tj * TILE + bx * 32 + lx] = v;
+    t[yy][lx] = v;
   }
+  if (tj == ti) return;
   __syncthreads();
-  if (tid == 0) {
-    if (J.dbg) {
-      unsigned long long t;
-      asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
-      J.dbg[3 * blockIdx.x + 1] = t;
+  for (int yy = ly; yy < 32; yy += 8)
+    Df[((int64_t)tj * TILE + bx * 32 + yy) * ldf + (int64_t)ti * TILE + by * 32 + lx] = t[lx][yy];
+}
+
+// The all-gather of D: every tile (ti, tj) of the full matrix Df is read from the window region of the
+// rank that owns it -- tile row ti when tj >= ti (owner of row ti under the zig-zag, local row position
+// = 2 * (ti / 2P) + (ti mod 2P >= P)), else the transpose of upper tile (tj, ti).  Regions hold the
+// owned tile rows with leading dimension Np.  Grid (nt, nt), 256 threads, 32 x 32 sub-blocks.
+__global__ void k_gather_pull(PeerPtrs regions, int32_t P, int32_t Np, int32_t *__restrict__ Df, int64_t ldf) {
+  __shared__ int32_t t[32][33];
+  const int ti = blockIdx.y, tj = blockIdx.x;
+  const int up = tj >= ti;
+  const int sr = up ? ti : tj, sc = up ? tj : ti;   // the authoritative tile (sr, sc), sc >= sr
+  const int o = sr % (2 * P);
+  const int rank = o < P ? o : 2 * P - 1 - o, pos = 2 * (sr / (2 * P)) + (o >= P ? 1 : 0);
+  const int32_t *src = reinterpret_cast<const int32_t *>(regions.p[rank]) + (int64_t)pos * TILE * Np + (int64_t)sc * TILE;
+  int32_t *dst = Df + (int64_t)ti * TILE * ldf + (int64_t)tj * TILE;
+  const int lx = threadIdx.x & 31, ly = threadIdx.x >> 5;
+  if (up) {
+    for (int i = threadIdx.x; i < TILE * TILE / 4; i += blockDim.x) {
+      const int r = i >> 5, c = (i & 31) * 4;
+      *reinterpret_cast<int4 *>(dst + (int64_t)r * ldf + c) = *reinterpret_cast<const int4 *>(src + (int64_t)r * Np + c);
     }
-    __threadfence();
-    if (atomicAdd(J.counter + 1, 1) == (int)gridDim.x - 1) {   // the last CTA resets the pair
-      J.counter[0] = 0;
-      J.counter[1] = 0;
-      __threadfence();
-    }
+    return;
+  }
+  for (int sb = 0; sb < 16; ++sb) {   // dst (r, c) = src (c, r)
+    const int bx = sb & 3, by = sb >> 2;
+    __syncthreads();
+    for (int yy = ly; yy < 32; yy += 8) t[yy][lx] = src[(int64_t)(bx * 32 + yy) * Np + by * 32 + lx];
+    __syncthreads();
+    for (int yy = ly; yy < 32; yy += 8) dst[(int64_t)(by * 32 + yy) * ldf + bx * 32 + lx] = t[lx][yy];
   }
 }
 
@@ -1097,7 +824,7 @@ __global__ void k_cc_init(int32_t *lab, int32_t n) {
   for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x)
     lab[v] = (int32_t)v;
 }
-__global__ void k_cc_hook16(const int32_t *u, const int32_t *v, int64_t E, int32_t *lab, int32_t *changed) {
+__global__ void k_cc_hook(const int32_t *u, const int32_t *v, int64_t E, int32_t *lab, int32_t *changed) {
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < E; i += (int64_t)gridDim.x * blockDim.x) {
     const int32_t a = lab[u[i]], b = lab[v[i]];
     if (a != b) {
@@ -1106,7 +833,7 @@ __global__ void k_cc_hook16(const int32_t *u, const int32_t *v, int64_t E, int32
     }
   }
 }
-__global__ void k_cc_jump16(int32_t *lab, int32_t n) {
+__global__ void k_cc_jump(int32_t *lab, int32_t n) {
   for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
     int32_t l = lab[v];
     while (lab[l] != l) l = lab[l];
@@ -1114,22 +841,54 @@ __global__ void k_cc_jump16(int32_t *lab, int32_t n) {
   }
 }
 
-int g_num_sms = 0;
+// EAR_DEBUG_RACE_US (test knob, tests/test_concurrency_gpu.py): a device-side spin of that length ahead
+// of each cross-tile launch keeps the device behind the host, and a host sleep of the same length
+// between recording the cross-tile event and the side stream's wait on it widens the window in which
+// another FW call on the device could interleave.  Per-call lookahead state makes the result immune.
+__global__ void k_debug_spin(long long ns) {
+  const long long t0 = clock64();
+  while (clock64() - t0 < ns * 2) {
+  }
+}
+int debug_race_us() {
+  const char *e = getenv("EAR_DEBUG_RACE_US");
+  return e ? atoi(e) : 0;
+}
+void debug_gpu_delay(cudaStream_t st) {
+  if (debug_race_us() > 0) k_debug_spin<<<1, 32, 0, st>>>((long long)debug_race_us() * 1000);
+}
+void debug_host_delay() {
+  if (debug_race_us() > 0) usleep((useconds_t)debug_race_us());
+}
+
+// ============================================================================== host side
+int grid_for(int64_t n) { return (int)std::max<int64_t>(1, std::min<int64_t>(ceil_div(n, 256), 148 * 16)); }
+
+int env_int(const char *name, int dflt) {
+  const char *e = getenv(name);
+  return e ? atoi(e) : dflt;
+}
+
 PFN_cuTensorMapEncodeTiled_v12000 g_encode = nullptr;
+std::once_flag g_encode_once;
 
 // 2-D tensor map over rows x cols (leading dimension ld elements of elem bytes) with a box_rows x 128 box
-ear_status_t make_map_t(CUtensorMap *map, CUtensorMapDataType dt, int elem, const void *base, int64_t rows,
-                        int64_t cols, int64_t ld, int box_rows) {
-  if (!g_encode) {
+ear_status_t make_map(CUtensorMap *map, int elem, const void *base, int64_t rows, int64_t cols, int64_t ld,
+                      int box_rows) {
+  std::call_once(g_encode_once, [] {
     cudaDriverEntryPointQueryResult q;
     void *fn = nullptr;
-    EAR_CUDA_TRY(cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q));
-    if (!fn || q != cudaDriverEntryPointSuccess) {
-      set_error("cuTensorMapEncodeTiled unavailable");
-      return EAR_ECUDA;
-    }
-    g_encode = (PFN_cuTensorMapEncodeTiled_v12000)fn;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      g_encode = (PFN_cuTensorMapEncodeTiled_v12000)fn;
+    cudaGetLastError();
+  });
+  if (!g_encode) {
+    set_error("cuTensorMapEncodeTiled unavailable");
+    return EAR_ECUDA;
   }
+  const CUtensorMapDataType dt = elem == 2 ? CU_TENSOR_MAP_DATA_TYPE_UINT16
+                                           : CU_TENSOR_MAP_DATA_TYPE_INT32;   // u32 operands: same bits
   cuuint64_t dims[2] = {(cuuint64_t)cols, (cuuint64_t)rows};
   cuuint64_t strides[1] = {(cuuint64_t)ld * elem};
   cuuint32_t box[2] = {(cuuint32_t)TILE, (cuuint32_t)box_rows};
@@ -1144,217 +903,124 @@ ear_status_t make_map_t(CUtensorMap *map, CUtensorMapDataType dt, int elem, cons
   return EAR_OK;
 }
 
-ear_status_t make_map(CUtensorMap *map, const int32_t *base, int64_t rows, int64_t cols, int64_t ld, int box_rows) {
-  return make_map_t(map, CU_TENSOR_MAP_DATA_TYPE_INT32, 4, base, rows, cols, ld, box_rows);
+template <class F>
+constexpr int smem_bytes() {
+  return F::STAGES * (F::A_BYTES + F::B_BYTES) + F::STAGES * 8 + F::STAGES * 4 + 8;
 }
 
-// The tile kernel's configuration, chosen by measurement on the B200 (cfg4, phase-3 share of the
-// VIADDMNMX peak; profiles/r01_fw_variants.txt): 64-deep k-chunks, a 2-stage TMA ring (128 KB), C
-// straight into registers, one 256-thread CTA per SM (161 registers, no spills), kk unrolled 16x.
-using FwTile = FwCfg<64, 2, 1, 16>;
-
-int fw_kc() { return FwTile::KC; }
-
-template <class CF>
-ear_status_t launch_cfg(const CUtensorMap &map, const TileJob &J, int64_t nblocks, cudaStream_t st) {
-  static bool attr = false;
-  if (!attr) {
-    EAR_CUDA_TRY(cudaFuncSetAttribute(k_fw_tiles<CF>, cudaFuncAttributeMaxDynamicSharedMemorySize, CF::SMEM));
-    attr = true;
-  }
-  int per_sm = 0;
-  EAR_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_fw_tiles<CF>, NT, CF::SMEM));
-  if (per_sm < 1) per_sm = 1;
-  const int64_t grid = std::min<int64_t>(nblocks, (int64_t)g_num_sms * per_sm);   // persistent
-  EAR_LAUNCH(k_fw_tiles<CF>, (unsigned)grid, NT, CF::SMEM, st)(map, J);
-  return EAR_OK;
-}
-
-ear_status_t launch_tiles(const CUtensorMap &map, TileJob J, int64_t nblocks, cudaStream_t st) {
-  if (!g_num_sms) {
-    int dev = 0;
-    EAR_CUDA_TRY(cudaGetDevice(&dev));
-    EAR_CUDA_TRY(cudaDeviceGetAttribute(&g_num_sms, cudaDevAttrMultiProcessorCount, dev));
-  }
-  if (nblocks <= 0) return EAR_OK;
-  J.ntiles = nblocks;
-  return launch_cfg<FwTile>(map, J, nblocks, st);
-}
-
-
-// Packed 16-bit tile kernel configuration, chosen by tools/sweep_fw16.py on the B200 (cfg4, 17
-// variants, profiles/r01_fw16_variants.jsonl): 128 threads with 16 x 8 values each, 32-deep k-chunks,
-// a 2-stage TMA ring (48 KB), 3 CTAs per SM, kk unrolled 16x; then (tools/lab_fw16_variant.sh,
-// profiles/r01u_fw16_refill.jsonl) last-arriver refills of the ring and an L2 prefetch of the next
-// C tile: 475.3 -> 471.6 ms on cfg4's plain FW (3-stage rings and 16-deep chunks measured slower);
-// then dynamic tile scheduling (k_fw_tiles16_dyn, the CTAs of an SM run at different speeds) and 4 CTA
-// slots left to the lookahead's pivot chain: 472.7 -> 445.9 ms (profiles/r01y_fw16_dyn.jsonl).
-using Fw16Tile = Fw16Cfg<32, 2, 3, 16, 128, 0, 1, 0, 1>;   // dynamic tile scheduling (k_fw_tiles16_dyn)
-using Fw16TileL = Fw16Cfg<32, 2, 3, 16, 128, 0, 1>;
-using Fw16TileL4 = Fw16Cfg<16, 4, 3, 16, 128, 0, 1>;
-using Fw16TileL3 = Fw16Cfg<32, 3, 3, 16, 128, 0, 1>;
-using Fw16TileLP = Fw16Cfg<32, 2, 3, 16, 128, 1, 1>;   // the static default before the tile counter
-using Fw16TileL3P = Fw16Cfg<32, 3, 3, 16, 128, 1, 1>;
-using Fw16TileS = Fw16Cfg<32, 2, 3, 16, 128, 1, 1, 1>;
-using Fw16TileS3 = Fw16Cfg<32, 3, 3, 16, 128, 1, 1, 1>;
-using Fw16TileD = Fw16Cfg<32, 2, 3, 16, 128, 1, 1, 0, 1>;
-using Fw16TileD0 = Fw16Cfg<32, 2, 3, 16, 128, 0, 1, 0, 1>;
-using Fw16TileD3 = Fw16Cfg<32, 3, 3, 16, 128, 0, 1, 0, 1>;
-using Fw16TileD16 = Fw16Cfg<16, 4, 3, 16, 128, 0, 1, 0, 1>;
-using Fw16TileD2x4 = Fw16Cfg<32, 4, 2, 16, 128, 0, 1, 0, 1>;
-using Fw16TileD2x3 = Fw16Cfg<32, 3, 2, 16, 128, 0, 1, 0, 1>;
-using Fw16TileDH = Fw16Cfg<32, 2, 3, 16, 128, 0, 1, 0, 1, 1>;
-
-// development knobs (tools/): EAR_FW16_LOOKAHEAD=0 disables the lookahead, EAR_FW16_RESERVE sets the
-// CTA slots the rest-of-round launch leaves free for the next round's pivot work (default 4: with the
-// persistent dynamically scheduled kernel no slot frees up before the launch drains; measured best,
-// profiles/r01y_fw16_dyn.jsonl), EAR_FW16_PRIO=0 gives the side stream normal priority
-int env_int(const char *name, int dflt) {
-  const char *e = getenv(name);
-  return e ? atoi(e) : dflt;
-}
-
-// the dynamic kernel's counter pair for launches on stream st: one pair per (device, stream), zeroed
-// once and reset by each launch's last CTA, so launches on one stream reuse it in order
-int32_t *dyn_counter(cudaStream_t st) {
-  static std::vector<std::pair<std::pair<int, cudaStream_t>, int32_t *>> pairs;
+// resident CTAs per SM of the tile kernel (per device, cached)
+template <class F>
+int tiles_per_sm() {
+  static int cache[64] = {};
+  static std::mutex mu;
   int dev = 0;
-  if (cudaGetDevice(&dev) != cudaSuccess) return nullptr;
-  for (auto &p : pairs)
-    if (p.first.first == dev && p.first.second == st) return p.second;
-  int32_t *c = nullptr;
-  if (cudaMalloc((void **)&c, 2 * sizeof(int32_t)) != cudaSuccess || cudaMemset(c, 0, 2 * sizeof(int32_t)) != cudaSuccess)
-    return nullptr;
-  pairs.push_back({{dev, st}, c});
-  return c;
+  cudaGetDevice(&dev);
+  std::lock_guard<std::mutex> lk(mu);
+  if (dev >= 0 && dev < 64 && cache[dev]) return cache[dev];
+  int per = 0;
+  if (smem_attr((const void *)k_fw_tiles<F>, smem_bytes<F>()) != cudaSuccess ||
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_fw_tiles<F>, F::NTH, smem_bytes<F>()) != cudaSuccess)
+    per = 0;
+  cudaGetLastError();
+  per = std::max(per, 1);
+  if (dev >= 0 && dev < 64) cache[dev] = per;
+  return per;
 }
 
-template <class CF>
-ear_status_t launch16_cfg(const CUtensorMap &mA, const CUtensorMap &mB, TileJob16 J, int64_t nblocks, cudaStream_t st,
-                          int reserve) {
-  auto kern = CF::kDYN ? k_fw_tiles16_dyn<CF> : k_fw_tiles16<CF>;
-  static bool attr = false;
-  if (!attr) {
-    EAR_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, CF::SMEM));
-    attr = true;
+template <class F>
+ear_status_t launch_tiles(const CUtensorMap &mA, const CUtensorMap &mB, TileJob J, int64_t ntiles, int32_t *counter,
+                          cudaStream_t st, int reserve = 0) {
+  if (ntiles <= 0) return EAR_OK;
+  if (ntiles >= 0xFFFFF) {
+    set_error("fw: %lld tiles in one launch exceed the tile kernel's 20-bit tile index", (long long)ntiles);
+    return EAR_EUNSUPPORTED;
   }
-  if (CF::kDYN) {
-    J.counter = dyn_counter(st);
-    if (!J.counter) {
-      set_error("fw16: no tile counter");
-      return EAR_ECUDA;
-    }
-  }
-  int per_sm = 0;
-  EAR_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, CF::kNTH, CF::SMEM));
-  if (per_sm < 1) per_sm = 1;
-  J.ntiles = nblocks;
-  const int64_t grid = std::min<int64_t>(nblocks, std::max<int64_t>(1, (int64_t)g_num_sms * per_sm - reserve));
-  // EAR_FW16_DBG=N (development): per-CTA start / end times and SM of the N-th launch, to stderr
-  static const int dbg_at = env_int("EAR_FW16_DBG", -1);
-  static int nlaunch = 0;
-  const bool dbg = dbg_at >= 0 && nlaunch++ == dbg_at;
-  if (dbg) EAR_CUDA_TRY(cudaMalloc((void **)&J.dbg, sizeof(unsigned long long) * 3 * grid));
-  EAR_LAUNCH(kern, (unsigned)grid, CF::kNTH, CF::SMEM, st)(mA, mB, J);
-  if (dbg) {
-    std::vector<unsigned long long> h(3 * grid);
-    EAR_CUDA_TRY(cudaStreamSynchronize(st));
-    EAR_CUDA_TRY(cudaMemcpy(h.data(), J.dbg, sizeof(unsigned long long) * 3 * grid, cudaMemcpyDeviceToHost));
-    cudaFree(J.dbg);
-    unsigned long long t0 = ~0ull;
-    for (int64_t b = 0; b < grid; ++b) t0 = std::min(t0, h[3 * b]);
-    fprintf(stderr, "FW16DBG launch %d grid %lld tiles %lld per_sm %d\n", dbg_at, (long long)grid, (long long)nblocks, per_sm);
-    for (int64_t b = 0; b < grid; ++b)
-      fprintf(stderr, "FW16DBG %lld %llu %llu %llu\n", (long long)b, h[3 * b] - t0, h[3 * b + 1] - t0, h[3 * b + 2]);
-  }
+  EAR_CUDA_TRY(smem_attr((const void *)k_fw_tiles<F>, smem_bytes<F>()));
+  J.ntiles = ntiles;
+  J.counter = counter;
+  const int64_t slots = (int64_t)num_sms() * tiles_per_sm<F>();
+  const int64_t grid = std::min<int64_t>(ntiles, std::max<int64_t>(1, slots - reserve));
+  EAR_LAUNCH(k_fw_tiles<F>, (unsigned)grid, F::NTH, smem_bytes<F>(), st)(mA, mB, J);
   return EAR_OK;
 }
-
-int fw16_kc() {
-  const int v = env_int("EAR_FW16_VARIANT", 0);
-  return v == 2 ? Fw16TileL4::kKC : v == 11 ? Fw16TileD16::kKC : Fw16Tile::kKC;
-}
-
-// EAR_FW16_VARIANT (development knob, tools/lab_fw16_*.sh): 0 = Fw16Tile; static tile assignment:
-// 1 = last-arriver refill, 2 = 4-stage ring of 16-deep chunks, 3 = 3-stage ring, 4 = refill + C prefetch
-// (the static default before), 5 = 3-stage + prefetch, 6/7 = polling waits; 8 = dynamic + C prefetch
-template <class CF>
-ear_status_t launch16(const CUtensorMap &mA, const CUtensorMap &mB, TileJob16 J, int64_t nblocks, cudaStream_t st,
-                      int reserve = 0) {
-  if (nblocks <= 0) return EAR_OK;
-  static const int variant = env_int("EAR_FW16_VARIANT", 0);
-  if (variant == 1) return launch16_cfg<Fw16TileL>(mA, mB, J, nblocks, st, reserve);
-  if (variant == 2) return launch16_cfg<Fw16TileL4>(mA, mB, J, nblocks, st, reserve);
-  if (variant == 3) return launch16_cfg<Fw16TileL3>(mA, mB, J, nblocks, st, reserve);
-  if (variant == 4) return launch16_cfg<Fw16TileLP>(mA, mB, J, nblocks, st, reserve);
-  if (variant == 5) return launch16_cfg<Fw16TileL3P>(mA, mB, J, nblocks, st, reserve);
-  if (variant == 6) return launch16_cfg<Fw16TileS>(mA, mB, J, nblocks, st, reserve);
-  if (variant == 7) return launch16_cfg<Fw16TileS3>(mA, mB, J, nblocks, st, reserve);
-  if (variant == 8) return launch16_cfg<Fw16TileD>(mA, mB, J, nblocks, st, reserve);
-  if (variant == 9) return launch16_cfg<Fw16TileD0>(mA, mB, J, nblocks, st, reserve);
-  if (variant == 10) return launch16_cfg<Fw16TileD3>(mA, mB, J, nblocks, st, reserve);
-  if (variant == 11) return launch16_cfg<Fw16TileD16>(mA, mB, J, nblocks, st, reserve);
-  if (variant == 12) return launch16_cfg<Fw16TileD2x4>(mA, mB, J, nblocks, st, reserve);
-  if (variant == 13) return launch16_cfg<Fw16TileD2x3>(mA, mB, J, nblocks, st, reserve);
-  if (variant == 14) return launch16_cfg<Fw16TileDH>(mA, mB, J, nblocks, st, reserve);
-  return launch16_cfg<CF>(mA, mB, J, nblocks, st, reserve);
-}
-
-int grid_for(int64_t n) { return (int)std::max<int64_t>(1, std::min<int64_t>(ceil_div(n, 256), 148 * 16)); }
 
 // CTA slots the rest-of-round launch leaves to the next round's pivot chain.  The persistent,
-// dynamically scheduled tile kernel frees no slot before it drains, so the chain's phase-2 tiles (one
-// pivot row, p2 tiles) run on the reserved slots alongside the rest (rest tiles): enough slots that
-// they finish no later, p2 / R <= rest / (slots - R).  EAR_FW16_RESERVE overrides (measured on cfg4's
-// single-GPU FW: 4 best, profiles/r01y_fw16_dyn.jsonl -- the rule gives 4 there, 5 on the re-reduced
-// BCC root piece and ~27 for a rank of 8, whose rest is 8x smaller; profiles/r01z_rank_timing_cfg4.jsonl).
+// dynamically scheduled tile kernel frees no slot before it drains, so the chain's phase-2 tiles (p2)
+// run on the reserved slots alongside the rest (rest tiles): enough slots that they finish no later,
+// p2 / R <= rest / (slots - R).  EAR_FW_RESERVE overrides (round 1 measured 4 best on cfg4's packed FW,
+// which is what the rule gives there, profiles/r01y_fw16_dyn.jsonl).
+template <class F>
 int lookahead_reserve(int64_t rest, int64_t p2) {
-  const int forced = env_int("EAR_FW16_RESERVE", -1);
+  const int forced = env_int("EAR_FW_RESERVE", -1);
   if (forced >= 0) return forced;
-  const int64_t slots = (int64_t)std::max(g_num_sms, 1) * 3;
+  const int64_t slots = (int64_t)num_sms() * tiles_per_sm<F>();
   const int64_t r = (slots * p2 + rest + p2 - 1) / std::max<int64_t>(rest + p2, 1);
   return (int)std::min<int64_t>(std::max<int64_t>(r, 1), slots / 2);
 }
 
-// the lookahead's side stream and events of the current device (created once, shared by the single-GPU
-// and the sharded packed FW; one FW call at a time per device)
-ear_status_t side_stream(cudaStream_t *side, cudaEvent_t *ev_cross, cudaEvent_t *ev_pivot) {
-  static cudaStream_t sides[64] = {};
-  static cudaEvent_t crosses[64] = {}, pivots[64] = {};
+// ---- per-call lookahead state: side stream, events and the precheck's mapped word, from a pool per
+// device (a context is held by one FW call from start to end: nothing is shared between calls)
+struct FwCtx {
+  int dev = -1;
+  cudaStream_t side = nullptr;
+  cudaEvent_t ev_cross = nullptr, ev_pivot = nullptr;
+  int32_t *h_word = nullptr;   // mapped pinned
+};
+std::mutex g_ctx_mu;
+std::vector<FwCtx *> g_ctx_free;
+
+ear_status_t ctx_acquire(FwCtx **out) {
   int dev = 0;
   EAR_CUDA_TRY(cudaGetDevice(&dev));
-  if (dev < 0 || dev >= 64) { set_error("side_stream: device %d out of range", dev); return EAR_EINVAL; }
-  if (!sides[dev]) {
-    int lo = 0, hi = 0;   // the pivot work gets the highest priority: its CTAs take the first free slots
-    EAR_CUDA_TRY(cudaDeviceGetStreamPriorityRange(&lo, &hi));
-    EAR_CUDA_TRY(cudaStreamCreateWithPriority(&sides[dev], cudaStreamNonBlocking, env_int("EAR_FW16_PRIO", 1) ? hi : lo));
-    EAR_CUDA_TRY(cudaEventCreateWithFlags(&crosses[dev], cudaEventDisableTiming));
-    EAR_CUDA_TRY(cudaEventCreateWithFlags(&pivots[dev], cudaEventDisableTiming));
+  {
+    std::lock_guard<std::mutex> lk(g_ctx_mu);
+    for (size_t i = 0; i < g_ctx_free.size(); ++i)
+      if (g_ctx_free[i]->dev == dev) {
+        *out = g_ctx_free[i];
+        g_ctx_free.erase(g_ctx_free.begin() + (long)i);
+        return EAR_OK;
+      }
   }
-  *side = sides[dev];
-  *ev_cross = crosses[dev];
-  *ev_pivot = pivots[dev];
+  FwCtx *c = new FwCtx;
+  c->dev = dev;
+  int lo = 0, hi = 0;   // the pivot chain gets the highest priority: its CTAs take the first free slots
+  cudaError_t e = cudaDeviceGetStreamPriorityRange(&lo, &hi);
+  if (e == cudaSuccess) e = cudaStreamCreateWithPriority(&c->side, cudaStreamNonBlocking, hi);
+  if (e == cudaSuccess) e = cudaEventCreateWithFlags(&c->ev_cross, cudaEventDisableTiming);
+  if (e == cudaSuccess) e = cudaEventCreateWithFlags(&c->ev_pivot, cudaEventDisableTiming);
+  if (e == cudaSuccess) e = cudaHostAlloc((void **)&c->h_word, sizeof(int32_t), cudaHostAllocMapped | cudaHostAllocPortable);
+  if (e != cudaSuccess) {
+    set_error("fw: lookahead context: %s", cudaGetErrorString(e));
+    delete c;
+    return EAR_ECUDA;
+  }
+  *out = c;
   return EAR_OK;
 }
+void ctx_release(FwCtx *c) {
+  if (!c) return;
+  std::lock_guard<std::mutex> lk(g_ctx_mu);
+  g_ctx_free.push_back(c);
+}
+struct CtxLease {
+  FwCtx *c = nullptr;
+  ~CtxLease() { ctx_release(c); }
+};
 
 // Cap precheck of the packed FW: one single-source SSSP row of reduced vertex 0 on a helper stream,
-// its eccentricity (a lower bound on the largest finite distance) read back asynchronously.  start()
-// does nothing without a plan, for a small FW (< 64 tiles) or with EAR_FW16_PRECHECK=0; hopeless()
-// waits for the row and says whether it reached the cap.  The row is exact and deterministic, so every
-// rank of a sharded FW takes the same decision without a collective.
+// its eccentricity (a lower bound on the largest finite distance) read back asynchronously into the
+// call's mapped word.  start() does nothing without a plan, for a small FW (< 64 tiles) or with
+// EAR_FW16_PRECHECK=0; hopeless() waits for the row and says whether it reached the cap.  The row is
+// exact and deterministic, so every rank of a sharded FW takes the same decision without a collective.
 struct Precheck {
   cudaStream_t hs = nullptr;
   cudaEvent_t ev = nullptr;
   int32_t *row = nullptr;
+  int32_t *h = nullptr;
   bool on = false;
-  static int32_t *host() {   // pinned, one per process (one FW at a time)
-    static int32_t *h = nullptr;
-    if (!h && cudaHostAlloc((void **)&h, sizeof(int32_t), cudaHostAllocMapped | cudaHostAllocPortable) != cudaSuccess)
-      h = nullptr;
-    return h;
-  }
-  void start(ear_plan_s *plan, int32_t Np, int32_t n_real, int nt) {
-    if (!plan || nt < 64 || env_int("EAR_FW16_PRECHECK", 1) == 0 || !host()) return;
+  void start(ear_plan_s *plan, int32_t Np, int32_t n_real, int nt, int32_t *h_word) {
+    h = h_word;
+    if (!plan || nt < 64 || env_int("EAR_FW16_PRECHECK", 1) == 0 || !h) return;
     on = cudaStreamCreateWithFlags(&hs, cudaStreamNonBlocking) == cudaSuccess &&
          cudaEventCreateWithFlags(&ev, cudaEventDisableTiming) == cudaSuccess &&
          cudaMallocAsync((void **)&row, sizeof(int32_t) * ((size_t)Np + 1), hs) == cudaSuccess &&
@@ -1362,12 +1028,11 @@ struct Precheck {
          sssp_rows(plan, row, Np, Np, 0, 1, nullptr, hs) == EAR_OK;
     if (on) {
       EAR_LAUNCH(k_row_far, grid_for(n_real), 256, 0, hs)(row, n_real, row + Np);
-      on = readback_direct(host(), row + Np, sizeof(int32_t), hs) == cudaSuccess &&
-           cudaEventRecord(ev, hs) == cudaSuccess;
+      on = readback_direct(h, row + Np, sizeof(int32_t), hs) == cudaSuccess && cudaEventRecord(ev, hs) == cudaSuccess;
     }
     if (!on) cudaGetLastError();
   }
-  bool hopeless() { return on && cudaEventSynchronize(ev) == cudaSuccess && *host() >= (int32_t)C16; }
+  bool hopeless() { return on && cudaEventSynchronize(ev) == cudaSuccess && *h >= (int32_t)C16; }
   void finish() {
     if (!hs) return;
     cudaStreamSynchronize(hs);
@@ -1380,144 +1045,505 @@ struct Precheck {
   ~Precheck() { finish(); }
 };
 
-// The packed 16-bit FW on a copy of D (see C16 above).  *done = false (D untouched) when a connected
-// pair reached the cap; the caller then runs the int32 FW.  Synchronises the stream once (the check).
-//
-// Lookahead: round k's phase 3 is split into the tiles of row/column k+1 (MODE_CROSS, first) and the
-// rest (MODE_REST).  As soon as the cross tiles are done, round k+1's pivot work -- phase 1 on tile
-// (k+1, k+1), the duplicated pivot row Pd, phase 2 on row k+1 -- runs on a side stream while the rest
-// of round k proceeds on the main stream (its launch leaves a few CTA slots free for it); round k+1's
-// phase 3 waits for both.  The two streams touch disjoint tiles (the rest skips rows/columns k, k+1)
-// and alternate between two Pd buffers, so the serial phases 1-2 leave the critical path.
-ear_status_t fw_single16(int32_t *D, int64_t ldd, int32_t Np, const int32_t *lab, int32_t n_real, bool *done,
-                         cudaStream_t st, ear_plan_s *plan) {
-  *done = false;
-  if (!g_num_sms) {
-    int dev = 0;
-    EAR_CUDA_TRY(cudaGetDevice(&dev));
-    EAR_CUDA_TRY(cudaDeviceGetAttribute(&g_num_sms, cudaDevAttrMultiProcessorCount, dev));
+// stream-ordered scratch of one FW call, freed in stream order at scope exit
+struct Scratch {
+  cudaStream_t st;
+  std::vector<void *> ptrs;
+  explicit Scratch(cudaStream_t s) : st(s) {}
+  template <class T>
+  bool get(T **p, size_t elems) {
+    *p = nullptr;
+    if (cudaMallocAsync((void **)p, sizeof(T) * std::max<size_t>(elems, 1), st) != cudaSuccess) {
+      cudaGetLastError();
+      *p = nullptr;
+      return false;
+    }
+    ptrs.push_back(*p);
+    return true;
   }
-  cudaStream_t side;
-  cudaEvent_t ev_cross, ev_pivot;
-  EAR_TRY(side_stream(&side, &ev_cross, &ev_pivot));
-  const bool lookahead = env_int("EAR_FW16_LOOKAHEAD", 1) != 0;
+  ~Scratch() {
+    for (void *p : ptrs) cudaFreeAsync(p, st);
+  }
+};
+
+// ============================================================================== single GPU
+// Single-GPU lookahead schedule for element policy F on the full symmetric matrix (int32: D itself;
+// packed: the capped u16 copy D16 with its duplicated pivot-row buffers Pd[2]).  Round k's phase 3 is
+// split into the tiles of row/column k+1 (MODE_CROSS, first) and the rest (MODE_REST); once the cross
+// tiles are done, round k+1's pivot chain -- phase 1 on tile (k+1, k+1), phase 2 on row k+1 (packed:
+// with its duplicated copies) -- runs on the call's side stream while the rest of round k proceeds
+// (leaving it a few CTA slots); round k+1's phase 3 waits for the chain.  The two streams touch disjoint
+// tiles (the rest skips rows/columns k, k+1; phase 2's mirrors land in column k+1).  With a precheck
+// (packed only) the schedule stops after round 3 when the cap is certainly reached (*hopeless).
+template <class F>
+ear_status_t fw_single_sched(typename F::E *D, int64_t ldd, int32_t Np, uint32_t *Pd, FwCtx *ctx, int32_t *cnt,
+                             cudaStream_t st, Precheck *pc, bool *hopeless) {
+  constexpr bool PACKED = sizeof(typename F::E) == 2;
+  using E = typename F::E;
   const int nt = Np / TILE;
   const double tile_ops = (double)TILE * TILE * TILE;
-  uint16_t *D16 = nullptr;
-  uint32_t *Pd = nullptr;   // two 128 x Np buffers (round parity)
-  int32_t *bad = nullptr;
-  if (cudaMallocAsync((void **)&D16, sizeof(uint16_t) * (size_t)Np * Np, st) != cudaSuccess ||
-      cudaMallocAsync((void **)&Pd, 2 * sizeof(uint32_t) * (size_t)TILE * Np, st) != cudaSuccess ||
-      cudaMallocAsync((void **)&bad, sizeof(int32_t), st) != cudaSuccess) {
-    cudaGetLastError();
-    if (D16) cudaFreeAsync(D16, st);
-    if (Pd) cudaFreeAsync(Pd, st);
-    return EAR_OK;   // no room for the 16-bit copy: the int32 path runs
-  }
-  const int KC = fw16_kc();
-  ear_status_t s = EAR_OK;
+  const bool lookahead = env_int("EAR_FW_LOOKAHEAD", 1) != 0;
+  *hopeless = false;
   CUtensorMap mA, mB[2];
-  s = make_map_t(&mA, CU_TENSOR_MAP_DATA_TYPE_UINT16, 2, D16, Np, Np, Np, KC);
-  for (int b = 0; b < 2 && s == EAR_OK; ++b)
-    s = make_map_t(&mB[b], CU_TENSOR_MAP_DATA_TYPE_UINT32, 4, Pd + (size_t)b * TILE * Np, TILE, Np, Np, KC);
+  EAR_TRY(make_map(&mA, (int)sizeof(E), D, Np, Np, ldd, F::KC));
+  if (PACKED)
+    for (int b = 0; b < 2; ++b) EAR_TRY(make_map(&mB[b], 4, Pd + (size_t)b * TILE * Np, TILE, Np, Np, F::KC));
   const int64_t ndup = (int64_t)TILE * (Np / 4);
-  if (s == EAR_OK) {
-    int sc = prof_begin(PK_FW16_CONV, st);
-    EAR_LAUNCH(k_to16, grid_for((int64_t)Np * (Np / 4)), 256, 0, st)(D, ldd, D16, Np);
-    prof_end(sc, st, 0);
-  }
-  // phases 1 and 2 of round k on stream q (Pd buffer k & 1)
+  int32_t *cnt_main = cnt, *cnt_side = cnt + 2;
+  // phases 1 and 2 of round k on stream q
   auto pivot = [&](int k, cudaStream_t q) -> ear_status_t {
-    uint16_t *P16 = D16 + (int64_t)k * TILE * Np;
-    uint32_t *Pk = Pd + (size_t)(k & 1) * TILE * Np;
-    const bool on_side = q != st;   // lookahead: overlapped with phase 3, reported apart
+    E *Pk = D + (int64_t)k * TILE * ldd;   // pivot row block
+    const bool on_side = q != st;          // lookahead: overlapped with phase 3, reported apart
     int s1 = prof_begin(on_side ? PK_FW_SIDE_P1 : PK_FW_P1, q);
-    EAR_LAUNCH(k_fw_phase1_16, 1, NT, 0, q)(P16 + (int64_t)k * TILE, Np);
+    if (PACKED)
+      EAR_LAUNCH(k_fw_phase1_16, 1, NT, 0, q)(reinterpret_cast<uint16_t *>(Pk) + (int64_t)k * TILE, ldd);
+    else
+      EAR_LAUNCH(k_fw_phase1, 1, NT, 0, q)(reinterpret_cast<int32_t *>(Pk) + (int64_t)k * TILE, ldd);
     prof_end(s1, q, tile_ops);
     int s2 = prof_begin(on_side ? PK_FW_SIDE_P2 : PK_FW_P2, q);
-    EAR_LAUNCH(k_dup16, grid_for(ndup), 256, 0, q)(P16, Np, Pk);   // B of phase 2: the pre-phase-2 row
-    TileJob16 J{D16, Np, k * TILE, k, nt, MODE_PIVOT_ROW, 1, 0};
-    EAR_TRY(launch16<Fw16Tile>(mA, mB[k & 1], J, nt - 1, q));
-    EAR_LAUNCH(k_dup16, grid_for(ndup), 256, 0, q)(P16, Np, Pk);   // B of phase 3
+    uint32_t *Pdk = Pd ? Pd + (size_t)(k & 1) * TILE * Np : nullptr;
+    if (PACKED)   // B of phase 2: the pre-phase-2 row, duplicated
+      EAR_LAUNCH(k_dup16, grid_for(ndup), 256, 0, q)(reinterpret_cast<const uint16_t *>(Pk), Np, Pdk);
+    TileJob J{D, ldd, k * TILE, PACKED ? 0 : k * TILE, k, nt, 0, MODE_PIVOT_ROW, 1};
+    EAR_TRY(launch_tiles<F>(mA, PACKED ? mB[k & 1] : mA, J, nt - 1, on_side ? cnt_side : cnt_main, q));
+    if (PACKED)   // B of phase 3
+      EAR_LAUNCH(k_dup16, grid_for(ndup), 256, 0, q)(reinterpret_cast<const uint16_t *>(Pk), Np, Pdk);
     prof_end(s2, q, (nt - 1) * tile_ops);
     return EAR_OK;
   };
-  if (s == EAR_OK && nt > 0) s = pivot(0, st);
-  // Cap precheck, overlapped with rounds 0-3: the exact distance row of reduced vertex 0 by one
-  // single-source SSSP on a helper stream.  Its eccentricity is a lower bound on the largest finite
-  // distance; when it already reaches the cap, a connected pair is capped for sure, so the packed FW
-  // is abandoned after round 3 instead of running to the end and being thrown away (cfg5: diameter
-  // ~42.8k).  Vertex 0 sits at a corner of the spatially coherent labellings, so its eccentricity is
-  // close to the diameter.  Only with a plan (plain FW, re-reduced pieces) and a large FW.
-  Precheck pc;
-  if (s == EAR_OK) pc.start(plan, Np, n_real, nt);
-  bool hopeless = false;
+  const int p3kind = PACKED ? PK_FW_P3_16 : PK_FW_P3;
+  ear_status_t s = nt > 0 ? pivot(0, st) : EAR_OK;
   for (int k = 0; k < nt && s == EAR_OK; ++k) {
-    if (k == 4 && pc.hopeless()) {   // rounds 0-3 (~4 ms at cfg4 sizes) cover the SSSP: the host rarely waits
-      hopeless = true;
+    if (k == 4 && pc && pc->hopeless()) {   // rounds 0-3 (~4 ms at cfg4 sizes) cover the SSSP
+      *hopeless = true;
       break;
     }
-    TileJob16 J{D16, Np, k * TILE, k, nt, MODE_UPPER, 1, 0};
-    const int64_t nup = (int64_t)(nt - 1) * nt / 2;
+    TileJob J{D, ldd, k * TILE, PACKED ? 0 : k * TILE, k, nt, 0, MODE_UPPER, 1};
+    const CUtensorMap &B = PACKED ? mB[k & 1] : mA;
     if (!lookahead || k + 1 == nt) {
-      int s3 = prof_begin(PK_FW_P3_16, st);
-      s = launch16<Fw16Tile>(mA, mB[k & 1], J, nup, st);
+      const int64_t nup = (int64_t)(nt - 1) * nt / 2;
+      int s3 = prof_begin(p3kind, st);
+      s = launch_tiles<F>(mA, B, J, nup, cnt_main, st);
       prof_end(s3, st, nup * tile_ops);
       if (s == EAR_OK && k + 1 < nt) s = pivot(k + 1, st);
       continue;
     }
-    int s3 = prof_begin(PK_FW_P3_16, st);
+    debug_gpu_delay(st);
+    int s3 = prof_begin(p3kind, st);
     J.mode = MODE_CROSS;
-    s = launch16<Fw16Tile>(mA, mB[k & 1], J, nt - 1, st);
+    s = launch_tiles<F>(mA, B, J, nt - 1, cnt_main, st);
     prof_end(s3, st, (nt - 1) * tile_ops);
     if (s != EAR_OK) break;
-    cudaError_t e = cudaEventRecord(ev_cross, st);
-    if (e == cudaSuccess) e = cudaStreamWaitEvent(side, ev_cross, 0);
-    if (e != cudaSuccess) { set_error("fw_single16: %s", cudaGetErrorString(e)); s = EAR_ECUDA; break; }
-    s = pivot(k + 1, side);
-    if (s != EAR_OK) break;
-    e = cudaEventRecord(ev_pivot, side);
-    if (e != cudaSuccess) { set_error("fw_single16: %s", cudaGetErrorString(e)); s = EAR_ECUDA; break; }
+    cudaError_t e = cudaEventRecord(ctx->ev_cross, st);
+    debug_host_delay();
+    if (e == cudaSuccess) e = cudaStreamWaitEvent(ctx->side, ctx->ev_cross, 0);
+    if (e != cudaSuccess) { set_error("fw_single: %s", cudaGetErrorString(e)); s = EAR_ECUDA; break; }
+    s = pivot(k + 1, ctx->side);
+    e = cudaEventRecord(ctx->ev_pivot, ctx->side);   // recorded even after an error: the main stream waits for it
+    if (s == EAR_OK && e != cudaSuccess) { set_error("fw_single: %s", cudaGetErrorString(e)); s = EAR_ECUDA; }
     J.mode = MODE_REST;
     const int64_t nrest = (int64_t)(nt - 2) * (nt - 1) / 2;
-    int s4 = prof_begin(PK_FW_P3_16, st);
-    s = launch16<Fw16Tile>(mA, mB[k & 1], J, nrest, st, lookahead_reserve(nrest, nt - 1));
+    int s4 = prof_begin(p3kind, st);
+    if (s == EAR_OK) s = launch_tiles<F>(mA, B, J, nrest, cnt_main, st, lookahead_reserve<F>(nrest, nt - 1));
     prof_end(s4, st, nrest * tile_ops);
-    if (s == EAR_OK) {
-      e = cudaStreamWaitEvent(st, ev_pivot, 0);
-      if (e != cudaSuccess) { set_error("fw_single16: %s", cudaGetErrorString(e)); s = EAR_ECUDA; }
-    }
+    e = cudaStreamWaitEvent(st, ctx->ev_pivot, 0);
+    if (s == EAR_OK && e != cudaSuccess) { set_error("fw_single: %s", cudaGetErrorString(e)); s = EAR_ECUDA; }
   }
-  if (s != EAR_OK) cudaStreamWaitEvent(st, ev_pivot, 0);   // never leave side work behind the frees
+  return s;
+}
+
+// The packed FW on a capped copy of D.  *done = false (D untouched) when a connected pair reached the
+// cap (or no memory for the copy); the caller then runs the int32 FW.  Synchronises the stream once.
+ear_status_t fw_single16(int32_t *D, int64_t ldd, int32_t Np, const int32_t *lab, int32_t n_real, bool *done,
+                         cudaStream_t st, ear_plan_s *plan, FwCtx *ctx, int32_t *cnt) {
+  *done = false;
+  Scratch sc(st);
+  uint16_t *D16 = nullptr;
+  uint32_t *Pd = nullptr;   // two 128 x Np buffers (round parity)
+  int32_t *bad = nullptr;
+  if (!sc.get(&D16, (size_t)Np * Np) || !sc.get(&Pd, 2 * (size_t)TILE * Np) || !sc.get(&bad, 1))
+    return EAR_OK;   // no room for the 16-bit copy: the int32 path runs
+  {
+    int c0 = prof_begin(PK_FW16_CONV, st);
+    EAR_LAUNCH(k_to16, grid_for((int64_t)Np * (Np / 4)), 256, 0, st)(D, ldd, D16, Np);
+    prof_end(c0, st, 0);
+  }
+  // Cap precheck, overlapped with rounds 0-3: the exact distance row of reduced vertex 0 by one
+  // single-source SSSP on a helper stream; its eccentricity is a lower bound on the largest finite
+  // distance, so when it already reaches the cap the packed FW is abandoned after round 3 instead of
+  // running to the end and being thrown away (cfg5: diameter ~42.8k).  Vertex 0 sits at a corner of the
+  // spatially coherent labellings, so its eccentricity is close to the diameter.
+  Precheck pc;
+  pc.start(plan, Np, n_real, Np / TILE, ctx->h_word);
+  bool hopeless = false;
+  ear_status_t s = fw_single_sched<Frag16>(D16, Np, Np, Pd, ctx, cnt, st, &pc, &hopeless);
+  if (s != EAR_OK) cudaStreamWaitEvent(st, ctx->ev_pivot, 0);   // never leave side work behind the frees
   pc.finish();
+  if (s != EAR_OK) return s;
+  if (hopeless) {
+    prof_fw16_precheck();
+    return EAR_OK;
+  }
   int32_t h_bad = 1;
-  if (s == EAR_OK && hopeless) prof_fw16_precheck();
-  if (s == EAR_OK && !hopeless) {
-    int sc = prof_begin(PK_FW16_CONV, st);
-    dev_memset(bad, 0, sizeof(int32_t), st);
-    EAR_LAUNCH(k_check16, grid_for((int64_t)Np * (Np / 8)), 256, 0, st)(D16, Np, lab, n_real, bad);
-    prof_end(sc, st, 0);
+  int c1 = prof_begin(PK_FW16_CONV, st);
+  EAR_CUDA_TRY(dev_memset(bad, 0, sizeof(int32_t), st));
+  EAR_LAUNCH(k_check16, grid_for((int64_t)Np * (Np / 8)), 256, 0, st)(D16, Np, lab, n_real, bad);
+  prof_end(c1, st, 0);
+  {
     Readback rb(st);
     cudaError_t e = rb.get(&h_bad, bad, sizeof(int32_t));
     if (e == cudaSuccess) e = rb.sync();
-    if (e != cudaSuccess) { set_error("fw_single16: %s", cudaGetErrorString(e)); s = EAR_ECUDA; }
+    if (e != cudaSuccess) { set_error("fw_single16: %s", cudaGetErrorString(e)); return EAR_ECUDA; }
   }
-  if (s == EAR_OK && h_bad == 0) {
-    int sc = prof_begin(PK_FW16_CONV, st);
+  if (h_bad == 0) {
+    int c2 = prof_begin(PK_FW16_CONV, st);
     EAR_LAUNCH(k_from16, grid_for((int64_t)Np * (Np / 4)), 256, 0, st)(D16, Np, D, ldd);
-    prof_end(sc, st, 0);
+    prof_end(c2, st, 0);
     *done = true;
   }
-  cudaFreeAsync(D16, st);
-  cudaFreeAsync(Pd, st);
-  cudaFreeAsync(bad, st);
-  if (s != EAR_OK) return s;
   EAR_CUDA_TRY(cudaGetLastError());
   return EAR_OK;
 }
 
+// ============================================================================== row-block sharding
+// Symmetric row-block sharding.  Tile rows are dealt to ranks in a zig-zag (rows r and 2P-1-r of every
+// group of 2P), so the UPPER tiles (ti, tj >= ti) -- the only authoritative ones -- balance across
+// ranks; rank r stores its owned tile rows (ascending) as 128-row blocks.  Round k's pivot chain:
+//   1. every rank copies its pieces of the pivot row block into L[k&1] (tile (k, j >= k) from the owner
+//      of row k, tiles (i < k, k) transposed from the owners of rows i);
+//   2. the owner of row k closes the pivot tile (phase 1) and pushes it into every peer's L[k&1];
+//   3. every rank applies phase 2 to ITS pieces only (MODE_PIECES, one product against the closed tile);
+//   4. every rank pushes its updated pieces into every rank's stage[k%3] and raises its flag -- the
+//      per-round broadcast: each rank receives exactly the rest of the pivot row block, once;
+//   5. once all flags are up, stage[k%3] is the complete updated block (packed: duplicated into the
+//      B operand), and each rank copies its pieces back into its storage.
+// Phase 3: every rank updates its owned upper tiles outside row/column k, both operands from stage.
+// Per-rank min-plus work is (N_r^3 / 2) / P: the single-GPU symmetric halving survives the sharding.
+// Buffer reuse is safe by the flag chain: a rank pushes round k+1's pieces only after it has every
+// rank's round-k pieces, which each peer sends only after its own round k-1 phase 3 -- so a stage
+// buffer is rewritten three rounds after its last reader, an L buffer two.
+std::vector<int32_t> shard_rows_of(int32_t nt, int32_t P, int32_t rank) {
+  std::vector<int32_t> rows;
+  for (int32_t ti = 0; ti < nt; ++ti) {
+    const int32_t o = ti % (2 * P);
+    if ((o < P ? o : 2 * P - 1 - o) == rank) rows.push_back(ti);
+  }
+  return rows;
+}
+
+int zz_owner(int32_t ti, int32_t P) {
+  const int32_t o = ti % (2 * P);
+  return o < P ? o : 2 * P - 1 - o;
+}
+
+struct Shard {
+  int32_t *S = nullptr;        // owned storage: nown x 128 rows x ldd (int32)
+  int64_t ldd = 0;
+  int32_t Np = 0, nt = 0, P = 1, rank = 0, nown = 0;
+  std::vector<int32_t> rows;
+  int32_t *d_rows = nullptr;
+  int64_t *d_pre = nullptr;
+  void pieces(int k, int *posk, int *mk, int *posk1 = nullptr) const {
+    *posk = -1;
+    *mk = 0;
+    if (posk1) *posk1 = -1;
+    for (int32_t r = 0; r < nown; ++r) {
+      if (rows[r] < k) ++*mk;
+      if (rows[r] == k) *posk = r;
+      if (posk1 && rows[r] == k + 1) *posk1 = r;
+    }
+  }
+};
+
+ear_status_t shard_setup(Shard *sh, int32_t *S, int64_t ldd, int32_t Np, int32_t P, int32_t rank, Scratch &sc) {
+  sh->S = S; sh->ldd = ldd; sh->Np = Np; sh->nt = Np / TILE; sh->P = P; sh->rank = rank;
+  sh->rows = shard_rows_of(sh->nt, P, rank);
+  sh->nown = (int32_t)sh->rows.size();
+  std::vector<int64_t> pre(sh->nown + 1, 0);
+  for (int32_t r = 0; r < sh->nown; ++r) pre[r + 1] = pre[r] + (sh->nt - sh->rows[r]);
+  if (!sc.get(&sh->d_rows, sh->nown) || !sc.get(&sh->d_pre, sh->nown + 1)) {
+    set_error("fw: out of device memory (shard tables)");
+    return EAR_ENOMEM;
+  }
+  if (sh->nown > 0) {
+    EAR_CUDA_TRY(cudaMemcpyAsync(sh->d_rows, sh->rows.data(), sizeof(int32_t) * sh->nown, cudaMemcpyHostToDevice, sc.st));
+    EAR_CUDA_TRY(cudaMemcpyAsync(sh->d_pre, pre.data(), sizeof(int64_t) * (sh->nown + 1), cudaMemcpyHostToDevice, sc.st));
+    EAR_CUDA_TRY(cudaStreamSynchronize(sc.st));   // host vectors are about to go out of scope
+  }
+  return EAR_OK;
+}
+
+// The sharded schedule for element policy F.  `sh` are the shards this process runs: one (its rank) with
+// a communicator, or P virtual ranks sharing the buffers on one device (comm == nullptr: the pushes then
+// land in the one shared stage and no flags are needed -- the same kernels and data movement otherwise).
+// Stor[r]: shard r's storage in F's element type (int32: sh[r]->S itself; packed: a narrowed copy), all
+// with leading dimension lds.  `solo` (rank timing): one rank's device work with the other ranks absent
+// -- no waits, no pushes to peers, garbage data.
+template <class F>
+ear_status_t fw_sharded_sched(std::vector<Shard *> &sh, std::vector<typename F::E *> &Stor, int64_t lds, int32_t Np,
+                              ear_comm_s *comm, FwCtx *ctx, int32_t *cnt, cudaStream_t st, Precheck *pc,
+                              bool *hopeless, bool solo) {
+  constexpr bool PACKED = sizeof(typename F::E) == 2;
+  using E = typename F::E;
+  const int nt = Np / TILE;
+  const int P = sh[0]->P;
+  const size_t R = sh.size();
+  const int64_t nblk = (int64_t)TILE * Np;
+  const bool lookahead = env_int("EAR_FW_LOOKAHEAD", 1) != 0;
+  const double tile_ops = (double)TILE * TILE * TILE;
+  *hopeless = false;
+  Scratch sc(st);
+  E *L[2] = {}, *stage[3] = {};
+  uint32_t *Ld = nullptr, *Pd = nullptr;
+  const bool real = comm && !solo;   // flags and pushes into the peers' windows
+  if (real) {
+    for (int b = 0; b < 2; ++b) L[b] = reinterpret_cast<E *>(comm_L(comm, comm->rank, b));
+    for (int b = 0; b < 3; ++b) stage[b] = reinterpret_cast<E *>(comm_stage(comm, comm->rank, b));
+  } else {
+    bool ok = true;
+    for (int b = 0; b < 2; ++b) ok = ok && sc.get(&L[b], nblk);
+    for (int b = 0; b < 3; ++b) ok = ok && sc.get(&stage[b], nblk);
+    if (!ok) { set_error("fw_sharded: out of device memory"); return EAR_ENOMEM; }
+  }
+  if (PACKED && (!sc.get(&Ld, nblk) || !sc.get(&Pd, 2 * nblk))) {
+    set_error("fw_sharded: out of device memory");
+    return EAR_ENOMEM;
+  }
+  CUtensorMap mL[2], mS[3], mLd, mPd[2];
+  for (int b = 0; b < 2; ++b) EAR_TRY(make_map(&mL[b], (int)sizeof(E), L[b], TILE, Np, Np, F::KC));
+  for (int b = 0; b < 3; ++b) EAR_TRY(make_map(&mS[b], (int)sizeof(E), stage[b], TILE, Np, Np, F::KC));
+  if (PACKED) {
+    EAR_TRY(make_map(&mLd, 4, Ld, TILE, Np, Np, F::KC));
+    for (int b = 0; b < 2; ++b) EAR_TRY(make_map(&mPd[b], 4, Pd + b * nblk, TILE, Np, Np, F::KC));
+  }
+  int32_t *cnt_main = cnt, *cnt_side = cnt + 2, *cnt_push = cnt + 4;
+  // destinations of this rank's pushes: every rank's stage[b] (comm), the shared one otherwise
+  auto stage_dsts = [&](int b) {
+    PeerPtrs d{};
+    if (real) {
+      d.n = comm->nranks;
+      for (int p = 0; p < comm->nranks; ++p) d.p[p] = comm_stage(comm, p, b);
+    } else {
+      d.n = 1;
+      d.p[0] = reinterpret_cast<char *>(stage[b]);
+    }
+    return d;
+  };
+  // round k's pivot chain on stream q
+  auto chain = [&](int k, cudaStream_t q) -> ear_status_t {
+    const bool on_side = q != st;
+    const int b = k & 1, s3 = k % 3;
+    int32_t *cq = on_side ? cnt_side : cnt_main;
+    for (size_t r = 0; r < R; ++r) {
+      int posk, mk;
+      sh[r]->pieces(k, &posk, &mk);
+      const int np = (posk >= 0 ? nt - k : 0) + mk;
+      if (np > 0)
+        EAR_LAUNCH(k_prow_xfer<E>, dim3(16, np), 256, 0, q)(Stor[r], lds, sh[r]->d_rows, k, nt, posk, L[b], Np, 0);
+    }
+    const int owner = zz_owner(k, P);
+    const bool mine = real ? comm->rank == owner : true;   // emulated / solo: the owner is local
+    int s1 = prof_begin(on_side ? PK_FW_SIDE_P1 : PK_FW_P1, q);
+    if (mine) {
+      if (PACKED)
+        EAR_LAUNCH(k_fw_phase1_16, 1, NT, 0, q)(reinterpret_cast<uint16_t *>(L[b]) + (int64_t)k * TILE, Np);
+      else
+        EAR_LAUNCH(k_fw_phase1, 1, NT, 0, q)(reinterpret_cast<int32_t *>(L[b]) + (int64_t)k * TILE, Np);
+    }
+    prof_end(s1, q, mine ? tile_ops : 0.0);
+    if (real && P > 1) {   // the closed pivot tile from its owner into every peer's L[b]
+      int sc1 = prof_begin(PK_COMM, q);
+      const uint64_t v = ++comm->seq_tile;
+      if (mine) {
+        PeerPtrs d{}, f{};
+        for (int p = 0; p < P; ++p)
+          if (p != comm->rank) {
+            d.p[d.n] = comm_L(comm, p, b);
+            f.p[f.n] = comm->peer[p];
+            ++d.n;
+            ++f.n;
+          }
+        // one "piece": column block k of the owner's L (posk = 0 with nt = k + 1 selects just it)
+        EAR_LAUNCH(k_push_pieces<E>, dim3(1, 4), 256, 0, q)(L[b], Np, k, k + 1, 0, 0, sh[0]->d_rows, d, cnt_push, f,
+                                                            SLOT_TILE + comm->rank, v);
+      } else {
+        EAR_TRY(comm_wait_one(comm, SLOT_TILE + owner, v, q));
+      }
+      prof_end(sc1, q, 0);
+    }
+    int s2 = prof_begin(on_side ? PK_FW_SIDE_P2 : PK_FW_P2, q);
+    if (PACKED) EAR_LAUNCH(k_dup16, grid_for(nblk / 4), 256, 0, q)(reinterpret_cast<uint16_t *>(L[b]), Np, Ld);
+    double p2 = 0;
+    for (size_t r = 0; r < R; ++r) {
+      int posk, mk;
+      sh[r]->pieces(k, &posk, &mk);
+      const int64_t n2 = mk + (posk >= 0 ? nt - 1 - k : 0);
+      if (n2 == 0) continue;
+      TileJob J2{L[b], Np, 0, 0, k, nt, k, MODE_PIECES, 0, 0, sh[r]->d_rows, sh[r]->d_pre, sh[r]->nown, mk, posk, -1};
+      EAR_TRY(launch_tiles<F>(mL[b], PACKED ? mLd : mL[b], J2, n2, cq, q));
+      p2 += (double)n2 * tile_ops;
+    }
+    prof_end(s2, q, p2);
+    int sc2 = prof_begin(PK_COMM, q);
+    const uint64_t vp = real ? ++comm->seq_pieces : 0;
+    for (size_t r = 0; r < R; ++r) {
+      int posk, mk;
+      sh[r]->pieces(k, &posk, &mk);
+      const int np = (posk >= 0 ? nt - k : 0) + mk;
+      if (np == 0 && !real) continue;
+      const PeerPtrs f = real ? comm_flags_all(comm) : PeerPtrs{};
+      EAR_LAUNCH(k_push_pieces<E>, dim3(std::max(np, 1), 4), 256, 0, q)(L[b], Np, k, nt, posk, mk, sh[r]->d_rows,
+                                                                        stage_dsts(s3), real ? cnt_push : nullptr, f,
+                                                                        SLOT_PIECES + (real ? comm->rank : 0), vp);
+    }
+    if (real) EAR_TRY(comm_wait(comm, SLOT_PIECES, vp, q));
+    prof_end(sc2, q, 0);
+    if (PACKED)
+      EAR_LAUNCH(k_dup16, grid_for(nblk / 4), 256, 0, q)(reinterpret_cast<uint16_t *>(stage[s3]), Np, Pd + b * nblk);
+    for (size_t r = 0; r < R; ++r) {
+      int posk, mk;
+      sh[r]->pieces(k, &posk, &mk);
+      const int np = (posk >= 0 ? nt - k : 0) + mk;
+      if (np > 0)
+        EAR_LAUNCH(k_prow_xfer<E>, dim3(16, np), 256, 0, q)(Stor[r], lds, sh[r]->d_rows, k, nt, posk, stage[s3], Np, 1);
+    }
+    return EAR_OK;
+  };
+  auto phase3 = [&](int k, int mode, cudaStream_t q, int reserve) -> ear_status_t {
+    const CUtensorMap &A = mS[k % 3], &B = PACKED ? mPd[k & 1] : mS[k % 3];
+    for (size_t r = 0; r < R; ++r) {
+      const Shard &s = *sh[r];
+      int posk, mk, posk1;
+      s.pieces(k, &posk, &mk, &posk1);
+      int64_t total = 0;
+      for (int32_t i = 0; i < s.nown; ++i) {
+        const int32_t ti = s.rows[i];
+        const int64_t all = ti == k ? 0 : (nt - ti) - (ti < k ? 1 : 0);
+        const int64_t cross = (ti == k + 1 ? nt - ti : 0) + (ti < k ? 1 : 0);
+        total += mode == MODE_LIST ? all : mode == MODE_LIST_CROSS ? cross : all - cross;
+      }
+      if (total == 0) continue;
+      const int res = reserve < 0 ? lookahead_reserve<F>(total, (nt - 1 + P - 1) / P) : reserve;
+      TileJob J{Stor[r], lds, 0, 0, k, nt, 0, mode, 0, 0, s.d_rows, s.d_pre, s.nown, mk, posk, posk1};
+      int s3 = prof_begin(PACKED ? PK_FW_P3_16 : PK_FW_P3, q);
+      EAR_TRY(launch_tiles<F>(A, B, J, total, cnt_main, q, res));
+      prof_end(s3, q, (double)total * tile_ops);
+    }
+    return EAR_OK;
+  };
+  ear_status_t s = chain(0, st);
+  for (int k = 0; k < nt && s == EAR_OK; ++k) {
+    if (k == 4 && pc && pc->hopeless()) {
+      *hopeless = true;
+      break;
+    }
+    if (!lookahead || k + 1 == nt) {
+      s = phase3(k, MODE_LIST, st, 0);
+      if (s == EAR_OK && k + 1 < nt) s = chain(k + 1, st);
+      continue;
+    }
+    debug_gpu_delay(st);
+    s = phase3(k, MODE_LIST_CROSS, st, 0);
+    if (s != EAR_OK) break;
+    cudaError_t e = cudaEventRecord(ctx->ev_cross, st);
+    debug_host_delay();
+    if (e == cudaSuccess) e = cudaStreamWaitEvent(ctx->side, ctx->ev_cross, 0);
+    if (e != cudaSuccess) { set_error("fw_sharded: %s", cudaGetErrorString(e)); s = EAR_ECUDA; break; }
+    s = chain(k + 1, ctx->side);
+    e = cudaEventRecord(ctx->ev_pivot, ctx->side);   // recorded even after an error: the main stream waits for it
+    if (s == EAR_OK && e != cudaSuccess) { set_error("fw_sharded: %s", cudaGetErrorString(e)); s = EAR_ECUDA; }
+    if (s == EAR_OK) s = phase3(k, MODE_LIST_REST, st, -1);
+    e = cudaStreamWaitEvent(st, ctx->ev_pivot, 0);
+    if (s == EAR_OK && e != cudaSuccess) { set_error("fw_sharded: %s", cudaGetErrorString(e)); s = EAR_ECUDA; }
+  }
+  if (s != EAR_OK) cudaStreamWaitEvent(st, ctx->ev_pivot, 0);
+  return s;
+}
+
+// Sharded FW over the shards `sh` (one rank with comm, or emulated ranks): the packed schedule first
+// (allow16; exact unless a connected pair reaches the cap -- checked over every rank's upper tiles and
+// agreed through the CHECK flags), the int32 schedule on the untouched int32 storage otherwise.
+ear_status_t fw_sharded_run(std::vector<Shard *> &sh, int32_t Np, ear_comm_s *comm, const int32_t *lab, int32_t n_real,
+                            bool allow16, cudaStream_t st, ear_plan_s *plan, bool solo, bool *used16) {
+  *used16 = false;
+  const int nt = Np / TILE;
+  const size_t R = sh.size();
+  FwCtx *ctx = nullptr;
+  EAR_TRY(ctx_acquire(&ctx));
+  CtxLease lease{ctx};
+  Scratch sc(st);
+  int32_t *cnt = nullptr;
+  if (!sc.get(&cnt, 8)) { set_error("fw_sharded: out of device memory"); return EAR_ENOMEM; }
+  EAR_CUDA_TRY(dev_memset(cnt, 0, 8 * sizeof(int32_t), st));
+  if (comm && !solo) EAR_TRY(comm_barrier(comm, st));   // every peer is done with the previous call's buffers
+  if (allow16 && nt >= 2) {
+    std::vector<uint16_t *> S16(R, nullptr);
+    int32_t *flag = nullptr;
+    bool ok = sc.get(&flag, 1);
+    for (size_t r = 0; r < R && ok; ++r) ok = sc.get(&S16[r], (size_t)std::max(sh[r]->nown, 1) * TILE * Np);
+    if (ok) {
+      int c0 = prof_begin(PK_FW16_CONV, st);
+      for (size_t r = 0; r < R; ++r)
+        if (sh[r]->nown > 0)
+          EAR_LAUNCH(k_to16r, grid_for((int64_t)sh[r]->nown * TILE * (Np / 4)), 256, 0, st)(
+              sh[r]->S, sh[r]->ldd, S16[r], Np, (int64_t)sh[r]->nown * TILE, Np);
+      prof_end(c0, st, 0);
+      Precheck pc;   // as fw_single16's; every rank decides the same
+      if (!solo) pc.start(plan, Np, n_real, nt, ctx->h_word);
+      bool hopeless = false;
+      ear_status_t s = fw_sharded_sched<Frag16>(sh, S16, Np, Np, comm, ctx, cnt, st, &pc, &hopeless, solo);
+      pc.finish();
+      EAR_TRY(s);
+      if (hopeless) {
+        prof_fw16_precheck();
+      } else if (solo) {
+        *used16 = true;
+        return EAR_OK;   // rank timing: no check, no result
+      } else {
+        int c1 = prof_begin(PK_FW16_CONV, st);
+        EAR_CUDA_TRY(dev_memset(flag, 0, sizeof(int32_t), st));
+        for (size_t r = 0; r < R; ++r)
+          if (sh[r]->nown > 0)
+            EAR_LAUNCH(k_check16_list, grid_for((int64_t)sh[r]->nown * TILE * (Np / 8)), 256, 0, st)(
+                S16[r], Np, sh[r]->d_rows, sh[r]->nown, Np, lab, n_real, flag);
+        prof_end(c1, st, 0);
+        if (comm && comm->nranks > 1) {   // OR of every rank's bit
+          const uint64_t v = ++comm->seq_check;
+          EAR_LAUNCH(k_check_push, 1, 32, 0, st)(flag, comm_flags_all(comm), SLOT_CHECK + comm->rank, v);
+          EAR_TRY(comm_wait(comm, SLOT_CHECK, v << 1, st));
+          EAR_LAUNCH(k_check_fold, 1, 32, 0, st)(reinterpret_cast<const uint64_t *>(comm->win) + SLOT_CHECK,
+                                                 comm->nranks, flag);
+        }
+        int32_t h_flag = -1;
+        Readback rb(st);
+        cudaError_t e = rb.get(&h_flag, flag, sizeof(int32_t));
+        if (e == cudaSuccess) e = rb.sync();
+        if (e != cudaSuccess) { set_error("fw_sharded: %s", cudaGetErrorString(e)); return EAR_ECUDA; }
+        if (h_flag == 0) {
+          int c2 = prof_begin(PK_FW16_CONV, st);
+          for (size_t r = 0; r < R; ++r)
+            if (sh[r]->nown > 0)
+              EAR_LAUNCH(k_from16r, grid_for((int64_t)sh[r]->nown * TILE * (Np / 4)), 256, 0, st)(
+                  S16[r], Np, sh[r]->S, sh[r]->ldd, (int64_t)sh[r]->nown * TILE, Np);
+          prof_end(c2, st, 0);
+          *used16 = true;
+          return EAR_OK;
+        }
+      }
+    } else {
+      cudaGetLastError();   // no room for the 16-bit copies: the int32 schedule runs
+    }
+  }
+  std::vector<int32_t *> S32(R);
+  for (size_t r = 0; r < R; ++r) S32[r] = sh[r]->S;
+  bool hopeless = false;
+  // every shard's storage has the same leading dimension (the callers allocate them alike)
+  return fw_sharded_sched<Frag32>(sh, S32, sh[0]->ldd, Np, comm, ctx, cnt, st, nullptr, &hopeless, solo);
+}
+
 }  // namespace
 
+// ============================================================================== internal API
 ear_status_t fw_init_D(const ear_plan_s *plan, int32_t *D, int64_t ldd, int32_t Np, int32_t row0, int32_t rows,
                        cudaStream_t st) {
   int64_t total = (int64_t)rows * (Np / 4);
@@ -1533,485 +1559,38 @@ ear_status_t fw_init_D(const ear_plan_s *plan, int32_t *D, int64_t ldd, int32_t 
   return EAR_OK;
 }
 
-// Single GPU: full symmetric D (Np x Np).  With allow16 the packed 16-bit FW runs first on a copy and
-// its result is kept when no connected pair (labels lab over [0, n_real), or one component when lab is
-// NULL) reached the 16-bit cap; otherwise, or without allow16, the int32 FW below runs.
+// Single GPU: full symmetric D (Np x Np).  With allow16 the packed FW runs first on a copy and its
+// result is kept when no connected pair (labels lab over [0, n_real), or one component when lab is
+// NULL) reached the cap; otherwise, or without allow16, the int32 schedule runs on D.
 ear_status_t fw_single(int32_t *D, int64_t ldd, int32_t Np, cudaStream_t st, const int32_t *lab, int32_t n_real,
                        bool allow16, ear_plan_s *plan) {
+  FwCtx *ctx = nullptr;
+  EAR_TRY(ctx_acquire(&ctx));
+  CtxLease lease{ctx};
+  Scratch sc(st);
+  int32_t *cnt = nullptr;   // tile counter pairs: main stream, side stream
+  if (!sc.get(&cnt, 4)) { set_error("fw_single: out of device memory"); return EAR_ENOMEM; }
+  EAR_CUDA_TRY(dev_memset(cnt, 0, 4 * sizeof(int32_t), st));
   if (allow16 && Np >= 2 * TILE) {
     bool done = false;
-    EAR_TRY(fw_single16(D, ldd, Np, lab, n_real, &done, st, plan));
+    EAR_TRY(fw_single16(D, ldd, Np, lab, n_real, &done, st, plan, ctx, cnt));
     prof_fw16(done);
     if (done) return EAR_OK;
   }
-  const int nt = Np / TILE;
-  const double tile_ops = (double)TILE * TILE * TILE;
-  CUtensorMap map;
-  EAR_TRY(make_map(&map, D, Np, Np, ldd, fw_kc()));
-  for (int k = 0; k < nt; ++k) {
-    int32_t *Pk = D + (int64_t)k * TILE * ldd;            // pivot row block
-    int s1 = prof_begin(PK_FW_P1, st);
-    EAR_LAUNCH(k_fw_phase1, 1, NT, 0, st)(Pk + (int64_t)k * TILE, ldd);
-    prof_end(s1, st, tile_ops);
-    TileJob J{D, ldd, k * TILE, k, nt, 0, nt, MODE_PIVOT_ROW, 1, 0};
-    int s2 = prof_begin(PK_FW_P2, st);
-    EAR_TRY(launch_tiles(map, J, nt - 1, st));
-    prof_end(s2, st, (nt - 1) * tile_ops);
-    J.mode = MODE_UPPER;
-    const int64_t nup = (int64_t)(nt - 1) * nt / 2;
-    int s3 = prof_begin(PK_FW_P3, st);
-    EAR_TRY(launch_tiles(map, J, nup, st));
-    prof_end(s3, st, nup * tile_ops);
-  }
-  EAR_CUDA_TRY(cudaGetLastError());
-  return EAR_OK;
-}
-
-// ---------------------------------------------------------------------------- row-block sharding
-// Symmetric row-block sharding.  Tile rows are dealt to ranks in a zig-zag (rows r and 2P-1-r of every
-// group of 2P), so the UPPER tiles (ti, tj >= ti) -- the only authoritative ones -- balance across
-// ranks; rank r stores its owned tile rows (ascending) as 128-row blocks.  Round k:
-//   1. every rank writes its pieces of the pivot row block into prow (tile (k, j >= k) from the owner
-//      of row k, tiles (i < k, k) transposed from the owners of rows i), INF elsewhere, and an
-//      all-reduce(MIN) over NCCL assembles the block on every rank;
-//   2. every rank closes the pivot tile (phase 1) and updates the pivot row block (phase 2) locally;
-//   3. owners copy the updated pivot pieces back into their storage;
-//   4. every rank updates its owned upper tiles outside row/column k (phase 3), both operands from prow.
-// Per-rank min-plus work is (N_r^3 / 2) / P + the redundant phase 1/2, i.e. the single-GPU symmetric
-// halving survives the sharding.  The final D is assembled by scattering every rank's upper tiles and
-// their mirrors into an INF-filled full matrix and one all-reduce(MIN).
-
-std::vector<int32_t> shard_rows(int32_t nt, int32_t P, int32_t rank) {
-  std::vector<int32_t> rows;
-  for (int32_t ti = 0; ti < nt; ++ti) {
-    const int32_t o = ti % (2 * P);
-    if ((o < P ? o : 2 * P - 1 - o) == rank) rows.push_back(ti);
-  }
-  return rows;
-}
-
-struct Shard {
-  int32_t *S = nullptr;        // owned storage: nown x 128 rows x ldd
-  int64_t ldd = 0;
-  int32_t Np = 0, nt = 0, P = 1, rank = 0, nown = 0;
-  std::vector<int32_t> rows;
-  int32_t *d_rows = nullptr;
-  int64_t *d_pre = nullptr;
-};
-
-static ear_status_t shard_setup(Shard *sh, int32_t *S, int64_t ldd, int32_t Np, int32_t P, int32_t rank,
-                                cudaStream_t st) {
-  sh->S = S; sh->ldd = ldd; sh->Np = Np; sh->nt = Np / TILE; sh->P = P; sh->rank = rank;
-  sh->rows = shard_rows(sh->nt, P, rank);
-  sh->nown = (int32_t)sh->rows.size();
-  std::vector<int64_t> pre(sh->nown + 1, 0);
-  for (int32_t r = 0; r < sh->nown; ++r) pre[r + 1] = pre[r] + (sh->nt - sh->rows[r]);
-  const size_t nr = std::max<int32_t>(sh->nown, 1);
-  EAR_CUDA_TRY(cudaMallocAsync((void **)&sh->d_rows, sizeof(int32_t) * nr, st));
-  EAR_CUDA_TRY(cudaMallocAsync((void **)&sh->d_pre, sizeof(int64_t) * (nr + 1), st));
-  if (sh->nown > 0) {
-    EAR_CUDA_TRY(cudaMemcpyAsync(sh->d_rows, sh->rows.data(), sizeof(int32_t) * sh->nown, cudaMemcpyHostToDevice, st));
-    EAR_CUDA_TRY(cudaMemcpyAsync(sh->d_pre, pre.data(), sizeof(int64_t) * (sh->nown + 1), cudaMemcpyHostToDevice, st));
-    EAR_CUDA_TRY(cudaStreamSynchronize(st));   // host vectors are about to go out of scope
-  }
-  return EAR_OK;
-}
-
-static void shard_free(Shard *sh, cudaStream_t st) {
-  if (sh->d_rows) cudaFreeAsync(sh->d_rows, st);
-  if (sh->d_pre) cudaFreeAsync(sh->d_pre, st);
-  sh->d_rows = nullptr; sh->d_pre = nullptr;
-}
-
-static ear_status_t fill(int32_t *p, int64_t n, int32_t v, cudaStream_t st) {
-  if (n <= 0) return EAR_OK;
-  EAR_LAUNCH(k_fill, (int)std::min<int64_t>(ceil_div(n, 256), 148 * 16), 256, 0, st)(p, n, v);
-  return EAR_OK;
-}
-
-// this rank's pieces of round k's pivot row block (see k_prow_xfer)
-static void shard_pieces(const Shard &sh, int k, int *posk, int *mk) {
-  *posk = -1;
-  *mk = 0;
-  for (int32_t r = 0; r < sh.nown; ++r) {
-    if (sh.rows[r] < k) ++*mk;
-    if (sh.rows[r] == k) *posk = r;
-  }
-}
-
-template <class TS, class TP>
-static ear_status_t shard_xfer_t(const Shard &sh, TS *S, int64_t ld, int k, TP *prow, int dir, cudaStream_t st) {
-  int posk, mk;
-  shard_pieces(sh, k, &posk, &mk);
-  const int np = (posk >= 0 ? sh.nt - k : 0) + mk;
-  if (np == 0) return EAR_OK;
-  EAR_LAUNCH((k_prow_xfer<TS, TP>), dim3(16, np), 256, 0, st)(S, ld, sh.d_rows, k, sh.nt, posk, prow, sh.Np, dir);
-  return EAR_OK;
-}
-
-static ear_status_t shard_xfer(const Shard &sh, int k, int32_t *prow, int dir, cudaStream_t st) {
-  return shard_xfer_t<int32_t, int32_t>(sh, sh.S, sh.ldd, k, prow, dir, st);
-}
-
-// phases 1 and 2 on the assembled pivot row block
-static ear_status_t shard_pivot(int32_t *prow, const CUtensorMap &map_prow, int32_t Np, int k, cudaStream_t st) {
-  const int nt = Np / TILE;
-  const double tile_ops = (double)TILE * TILE * TILE;
-  int s1 = prof_begin(PK_FW_P1, st);
-  EAR_LAUNCH(k_fw_phase1, 1, NT, 0, st)(prow + (int64_t)k * TILE, Np);
-  prof_end(s1, st, tile_ops);
-  TileJob J{prow, Np, 0, k, nt, k, 1, MODE_PIVOT_ROW, 0, 0, nullptr, nullptr, 0, 0, -1};
-  int s2 = prof_begin(PK_FW_P2, st);
-  EAR_TRY(launch_tiles(map_prow, J, nt - 1, st));
-  prof_end(s2, st, (nt - 1) * tile_ops);
-  return EAR_OK;
-}
-
-static ear_status_t shard_phase3(const Shard &sh, const CUtensorMap &map_prow, int k, cudaStream_t st) {
-  int mk = 0, posk = -1;
-  for (int32_t r = 0; r < sh.nown; ++r) {
-    if (sh.rows[r] < k) ++mk;
-    if (sh.rows[r] == k) posk = r;
-  }
-  int64_t total = 0;
-  for (int32_t r = 0; r < sh.nown; ++r) {
-    const int32_t ti = sh.rows[r];
-    total += ti == k ? 0 : (sh.nt - ti) - (ti < k ? 1 : 0);
-  }
-  TileJob J{sh.S, sh.ldd, 0, k, sh.nt, 0, sh.nown, MODE_LIST, 0, 0, sh.d_rows, sh.d_pre, sh.nown, mk, posk};
-  int s3 = prof_begin(PK_FW_P3, st);
-  EAR_TRY(launch_tiles(map_prow, J, total, st));
-  prof_end(s3, st, (double)total * TILE * TILE * TILE);
-  return EAR_OK;
-}
-
-ear_status_t fw_sharded(int32_t *S, int64_t ldd, int32_t Np, ear_comm_s *comm, cudaStream_t st) {
-  Shard sh;
-  EAR_TRY(shard_setup(&sh, S, ldd, Np, comm->nranks, comm->rank, st));
-  int32_t *prow = nullptr;
-  EAR_CUDA_TRY(cudaMallocAsync((void **)&prow, sizeof(int32_t) * (size_t)TILE * Np, st));
-  CUtensorMap map_prow;
-  ear_status_t status = make_map(&map_prow, prow, TILE, Np, Np, fw_kc());
-  for (int k = 0; k < sh.nt && status == EAR_OK; ++k) {
-    status = fill(prow, (int64_t)TILE * Np, INF, st);
-    if (status == EAR_OK) status = shard_xfer(sh, k, prow, 0, st);
-    if (status == EAR_OK) {
-      int sc = prof_begin(PK_COMM, st);
-      status = comm_allreduce_min(comm, prow, (int64_t)TILE * Np, st);
-      prof_end(sc, st, 0);
-    }
-    if (status == EAR_OK) status = shard_pivot(prow, map_prow, Np, k, st);
-    if (status == EAR_OK) status = shard_xfer(sh, k, prow, 1, st);
-    if (status == EAR_OK) status = shard_phase3(sh, map_prow, k, st);
-  }
-  cudaFreeAsync(prow, st);
-  shard_free(&sh, st);
-  if (status != EAR_OK) return status;
-  EAR_CUDA_TRY(cudaGetLastError());
-  return EAR_OK;
-}
-
-// ---------------------------------------------------------------- 16-bit row-block sharding
-// The sharded schedule above on packed 16-bit owned rows (the cap C16 and its exactness argument are
-// those of fw_single16).  The exchange stays int32 -- NCCL has no 16-bit MIN: the owned u16 pieces are
-// widened into the INF-filled int32 pivot row block and all-reduced; the block is narrowed back to u16
-// (values <= C16, so exactly the capped values) and closed by the packed phases 1-2 of fw_single16's
-// pivot() -- phase 1 on the pivot tile, phase 2 as one product against the duplicated pre-phase-2 row --
-// then scattered back to the owners; its duplicated copy is the B operand of the packed phase-3
-// kernel, which updates the owned u16 rows (MODE_LIST).
-// comm == nullptr: the shards are virtual ranks on this device sharing the block (their pieces are
-// disjoint, so no exchange is needed).  The range check runs over every rank's owned upper tiles and
-// is MIN-reduced; *done = false leaves the int32 owned storage untouched for the int32 schedule.
-static ear_status_t phase3_16(const Shard &sh, uint16_t *S16, const CUtensorMap &mA, const CUtensorMap &mB, int k,
-                              int mode, cudaStream_t st, int reserve = 0) {   // reserve < 0: lookahead_reserve
-  int mk = 0, posk = -1, posk1 = -1;
-  int64_t total = 0;
-  for (int32_t r = 0; r < sh.nown; ++r) {
-    const int32_t ti = sh.rows[r];
-    if (ti < k) ++mk;
-    if (ti == k) posk = r;
-    if (ti == k + 1) posk1 = r;
-  }
-  for (int32_t r = 0; r < sh.nown; ++r) {
-    const int32_t ti = sh.rows[r];
-    const int64_t all = ti == k ? 0 : (sh.nt - ti) - (ti < k ? 1 : 0);
-    const int64_t cross = (ti == k + 1 ? sh.nt - ti : 0) + (ti < k ? 1 : 0);
-    total += mode == MODE_LIST ? all : mode == MODE_LIST_CROSS ? cross : all - cross;
-  }
-  if (total == 0) return EAR_OK;
-  if (reserve < 0) reserve = lookahead_reserve(total, (sh.nt - 1 + sh.P - 1) / sh.P);   // owner-side phase 2
-  TileJob16 J{S16, sh.Np, 0, k, sh.nt, mode, 0, 0, sh.d_rows, sh.d_pre, sh.nown, mk, posk};
-  J.posk1 = posk1;
-  int s3 = prof_begin(PK_FW_P3_16, st);
-  EAR_TRY(launch16<Fw16Tile>(mA, mB, J, total, st, reserve));
-  prof_end(s3, st, (double)total * TILE * TILE * TILE);
-  return EAR_OK;
-}
-
-// Lookahead (as fw_single16's): round k's phase 3 is split into the owned tiles of row/column k+1
-// (MODE_LIST_CROSS, first) and the rest (MODE_LIST_REST); once the cross tiles are done, round k+1's
-// pivot chain -- pieces into the exchange block, the all-reduce, narrowing, phases 1-2, scatter back --
-// runs on the side stream (NCCL included) while the rest of round k proceeds; the two touch disjoint
-// tiles, the narrowed block and its duplicate alternate between two buffers by round parity, and round
-// k+1's phase 3 waits for the chain.
-static ear_status_t fw_sharded16(std::vector<Shard *> &sh, int32_t Np, ear_comm_s *comm, const int32_t *lab,
-                                 int32_t n_real, bool *done, cudaStream_t st, bool timing_only = false,
-                                 ear_plan_s *plan = nullptr) {
-  *done = false;
-  const int nt = Np / TILE;
-  if (nt < 2) return EAR_OK;
-  if (!g_num_sms) {
-    int dev = 0;
-    EAR_CUDA_TRY(cudaGetDevice(&dev));
-    EAR_CUDA_TRY(cudaDeviceGetAttribute(&g_num_sms, cudaDevAttrMultiProcessorCount, dev));
-  }
-  cudaStream_t side;
-  cudaEvent_t ev_cross, ev_pivot;
-  EAR_TRY(side_stream(&side, &ev_cross, &ev_pivot));
-  const bool lookahead = env_int("EAR_FW16_LOOKAHEAD", 1) != 0;
-  const size_t R = sh.size();
-  std::vector<uint16_t *> S16(R, nullptr);
-  int32_t *prow = nullptr, *flag = nullptr;
-  uint16_t *p16 = nullptr;   // two 128 x Np buffers (round parity), as Pd
-  uint32_t *Pd = nullptr;
-  uint16_t *L16 = nullptr, *ptile = nullptr;   // this rank's pivot-row pieces; the broadcast pivot tile
-  uint32_t *Ld = nullptr;                      // L16 duplicated (phase-2 B operand)
-  const int P = comm ? comm->nranks : (int)sh.size();
-  bool ok = cudaMallocAsync((void **)&prow, sizeof(int32_t) * (size_t)TILE * Np, st) == cudaSuccess &&
-            cudaMallocAsync((void **)&L16, sizeof(uint16_t) * (size_t)TILE * Np, st) == cudaSuccess &&
-            cudaMallocAsync((void **)&Ld, sizeof(uint32_t) * (size_t)TILE * Np, st) == cudaSuccess &&
-            cudaMallocAsync((void **)&ptile, sizeof(uint16_t) * TILE * TILE, st) == cudaSuccess &&
-            cudaMallocAsync((void **)&p16, 2 * sizeof(uint16_t) * (size_t)TILE * Np, st) == cudaSuccess &&
-            cudaMallocAsync((void **)&Pd, 2 * sizeof(uint32_t) * (size_t)TILE * Np, st) == cudaSuccess &&
-            cudaMallocAsync((void **)&flag, sizeof(int32_t), st) == cudaSuccess;
-  for (size_t r = 0; r < R && ok; ++r)
-    ok = cudaMallocAsync((void **)&S16[r], sizeof(uint16_t) * (size_t)std::max(sh[r]->nown, 1) * TILE * Np, st) ==
-         cudaSuccess;
-  auto release = [&]() {
-    for (size_t r = 0; r < R; ++r)
-      if (S16[r]) cudaFreeAsync(S16[r], st);
-    if (prow) cudaFreeAsync(prow, st);
-    if (p16) cudaFreeAsync(p16, st);
-    if (Pd) cudaFreeAsync(Pd, st);
-    if (L16) cudaFreeAsync(L16, st);
-    if (Ld) cudaFreeAsync(Ld, st);
-    if (ptile) cudaFreeAsync(ptile, st);
-    if (flag) cudaFreeAsync(flag, st);
-  };
-  if (!ok) {   // no room for the 16-bit copies: the int32 schedule runs
-    cudaGetLastError();
-    release();
-    return EAR_OK;
-  }
-  const int KC = fw16_kc();
-  const int64_t nblk = (int64_t)TILE * Np;
-  CUtensorMap mA[2], mB[2], mL, mLd;
-  ear_status_t s = make_map_t(&mL, CU_TENSOR_MAP_DATA_TYPE_UINT16, 2, L16, TILE, Np, Np, KC);
-  if (s == EAR_OK) s = make_map_t(&mLd, CU_TENSOR_MAP_DATA_TYPE_UINT32, 4, Ld, TILE, Np, Np, KC);
-  for (int b = 0; b < 2 && s == EAR_OK; ++b) {
-    s = make_map_t(&mA[b], CU_TENSOR_MAP_DATA_TYPE_UINT16, 2, p16 + b * nblk, TILE, Np, Np, KC);
-    if (s == EAR_OK) s = make_map_t(&mB[b], CU_TENSOR_MAP_DATA_TYPE_UINT32, 4, Pd + b * nblk, TILE, Np, Np, KC);
-  }
-  if (s == EAR_OK) {
-    int sc = prof_begin(PK_FW16_CONV, st);
-    for (size_t r = 0; r < R; ++r)
-      if (sh[r]->nown > 0)
-        EAR_LAUNCH(k_to16r, grid_for((int64_t)sh[r]->nown * TILE * (Np / 4)), 256, 0, st)(
-            sh[r]->S, sh[r]->ldd, S16[r], Np, (int64_t)sh[r]->nown * TILE, Np);
-    prof_end(sc, st, 0);
-  }
-  // round k's pivot chain on stream q, with the phase 2 done by the owners of the pieces:
-  //   every rank copies its pieces of the pivot row block into L (u16, C16 elsewhere -- above every
-  //   capped value, so the MIN exchange ignores it); the owner of row k closes the pivot tile in L
-  //   (phase 1) and broadcasts it (32 KB); every rank applies phase 2 to ITS pieces only (MODE_PIECES,
-  //   B = L duplicated before phase 2, as fw_single16's single-product phase 2); the pieces are
-  //   widened and all-reduced (MIN) into the full phase-2-complete block, which is narrowed into the
-  //   A operand of phase 3 (buffer k & 1), duplicated into its B operand and scattered back to the
-  //   owners.  No phase 2 is computed twice: each tile of the pivot row is updated by its contributor.
-  auto chain = [&](int k, cudaStream_t q) -> ear_status_t {
-    const bool on_side = q != st;
-    uint16_t *P16 = p16 + (k & 1) * nblk;
-    uint32_t *Pk = Pd + (k & 1) * nblk;
-    EAR_LAUNCH(k_fill16, grid_for(nblk / 2), 256, 0, q)(L16, nblk / 2, (uint32_t)C16 * 0x10001u);
-    for (size_t r = 0; r < R; ++r)
-      if (sh[r]->nown > 0) EAR_TRY((shard_xfer_t<uint16_t, uint16_t>(*sh[r], S16[r], Np, k, L16, 0, q)));
-    const int o = k % (2 * P), owner = o < P ? o : 2 * P - 1 - o;
-    const bool mine = comm ? comm->rank == owner : true;   // emulated: some shard owns it
-    int s1 = prof_begin(on_side ? PK_FW_SIDE_P1 : PK_FW_P1, q);
-    if (mine) EAR_LAUNCH(k_fw_phase1_16, 1, NT, 0, q)(L16 + (int64_t)k * TILE, Np);
-    prof_end(s1, q, mine ? (double)TILE * TILE * TILE : 0.0);
-    if (comm && P > 1) {   // the closed pivot tile from its owner
-      int sc = prof_begin(PK_COMM, q);
-      const size_t pitch = sizeof(uint16_t) * Np, w = sizeof(uint16_t) * TILE;
-      if (mine) EAR_CUDA_TRY(cudaMemcpy2DAsync(ptile, w, L16 + (int64_t)k * TILE, pitch, w, TILE, cudaMemcpyDeviceToDevice, q));
-      EAR_TRY(comm_bcast(comm, reinterpret_cast<int32_t *>(ptile), TILE * TILE / 2, owner, q));
-      if (!mine) EAR_CUDA_TRY(cudaMemcpy2DAsync(L16 + (int64_t)k * TILE, pitch, ptile, w, w, TILE, cudaMemcpyDeviceToDevice, q));
-      prof_end(sc, q, 0);
-    }
-    int s2 = prof_begin(on_side ? PK_FW_SIDE_P2 : PK_FW_P2, q);
-    EAR_LAUNCH(k_dup16, grid_for(nblk / 4), 256, 0, q)(L16, Np, Ld);
-    double p2 = 0;
-    for (size_t r = 0; r < R; ++r) {
-      int posk, mk;
-      shard_pieces(*sh[r], k, &posk, &mk);
-      const int64_t n2 = mk + (posk >= 0 ? nt - 1 - k : 0);
-      if (n2 == 0) continue;
-      TileJob16 J2{L16, Np, 0, k, nt, MODE_PIECES, 0, 0, sh[r]->d_rows, sh[r]->d_pre, sh[r]->nown, mk, posk};
-      EAR_TRY(launch16<Fw16Tile>(mL, mLd, J2, n2, q));
-      p2 += (double)n2 * TILE * TILE * TILE;
-    }
-    prof_end(s2, q, p2);
-    EAR_LAUNCH(k_widen16, grid_for(nblk / 4), 256, 0, q)(L16, prow, nblk);
-    if (comm) {
-      int sc = prof_begin(PK_COMM, q);
-      EAR_TRY(comm_allreduce_min(comm, prow, nblk, q));
-      prof_end(sc, q, 0);
-    }
-    EAR_LAUNCH(k_prow_to16, grid_for(nblk / 4), 256, 0, q)(prow, P16, Pk, nblk);
-    for (size_t r = 0; r < R; ++r)
-      if (sh[r]->nown > 0) EAR_TRY((shard_xfer_t<uint16_t, uint16_t>(*sh[r], S16[r], Np, k, P16, 1, q)));
-    return EAR_OK;
-  };
-  if (s == EAR_OK) s = chain(0, st);
-  Precheck pc;   // as fw_single16's; every rank decides the same
-  if (s == EAR_OK && !timing_only) pc.start(plan, Np, n_real, nt);
   bool hopeless = false;
-  for (int k = 0; k < nt && s == EAR_OK; ++k) {
-    if (k == 4 && pc.hopeless()) {
-      hopeless = true;
-      break;
-    }
-    const CUtensorMap &A = mA[k & 1], &B = mB[k & 1];
-    if (!lookahead || k + 1 == nt) {
-      for (size_t r = 0; r < R && s == EAR_OK; ++r) s = phase3_16(*sh[r], S16[r], A, B, k, MODE_LIST, st);
-      if (s == EAR_OK && k + 1 < nt) s = chain(k + 1, st);
-      continue;
-    }
-    for (size_t r = 0; r < R && s == EAR_OK; ++r) s = phase3_16(*sh[r], S16[r], A, B, k, MODE_LIST_CROSS, st);
-    if (s != EAR_OK) break;
-    cudaError_t e = cudaEventRecord(ev_cross, st);
-    if (e == cudaSuccess) e = cudaStreamWaitEvent(side, ev_cross, 0);
-    if (e != cudaSuccess) { set_error("fw_sharded16: %s", cudaGetErrorString(e)); s = EAR_ECUDA; break; }
-    s = chain(k + 1, side);
-    e = cudaEventRecord(ev_pivot, side);   // recorded even after an error: the main stream waits for it
-    if (s == EAR_OK && e != cudaSuccess) { set_error("fw_sharded16: %s", cudaGetErrorString(e)); s = EAR_ECUDA; }
-    for (size_t r = 0; r < R && s == EAR_OK; ++r)
-      s = phase3_16(*sh[r], S16[r], A, B, k, MODE_LIST_REST, st, -1);
-    e = cudaStreamWaitEvent(st, ev_pivot, 0);
-    if (s == EAR_OK && e != cudaSuccess) { set_error("fw_sharded16: %s", cudaGetErrorString(e)); s = EAR_ECUDA; }
-  }
-  pc.finish();
-  if (s == EAR_OK && hopeless) {   // the int32 schedule runs on the untouched int32 rows
-    prof_fw16_precheck();
-    release();
-    EAR_CUDA_TRY(cudaGetLastError());
-    return EAR_OK;
-  }
-  int32_t h_flag = -1;
-  if (s == EAR_OK && timing_only) {   // apsp_reduced_rank_timing: no check, no result
-    release();
-    EAR_CUDA_TRY(cudaGetLastError());
-    return EAR_OK;
-  }
-  if (s == EAR_OK) {
-    int sc = prof_begin(PK_FW16_CONV, st);
-    dev_memset(flag, 0, sizeof(int32_t), st);
-    for (size_t r = 0; r < R; ++r)
-      if (sh[r]->nown > 0)
-        EAR_LAUNCH(k_check16_list, grid_for((int64_t)sh[r]->nown * TILE * (Np / 8)), 256, 0, st)(
-            S16[r], Np, sh[r]->d_rows, sh[r]->nown, Np, lab, n_real, flag);
-    prof_end(sc, st, 0);
-    if (comm) s = comm_allreduce_min(comm, flag, 1, st);
-    Readback rb(st);
-    cudaError_t e = rb.get(&h_flag, flag, sizeof(int32_t));
-    if (e == cudaSuccess) e = rb.sync();
-    if (s == EAR_OK && e != cudaSuccess) { set_error("fw_sharded16: %s", cudaGetErrorString(e)); s = EAR_ECUDA; }
-  }
-  if (s == EAR_OK && h_flag == 0) {
-    int sc = prof_begin(PK_FW16_CONV, st);
-    for (size_t r = 0; r < R; ++r)
-      if (sh[r]->nown > 0)
-        EAR_LAUNCH(k_from16r, grid_for((int64_t)sh[r]->nown * TILE * (Np / 4)), 256, 0, st)(
-            S16[r], Np, sh[r]->S, sh[r]->ldd, (int64_t)sh[r]->nown * TILE, Np);
-    prof_end(sc, st, 0);
-    *done = true;
-  }
-  release();
-  if (s != EAR_OK) return s;
+  ear_status_t s = fw_single_sched<Frag32>(D, ldd, Np, nullptr, ctx, cnt, st, nullptr, &hopeless);
+  if (s != EAR_OK) cudaStreamWaitEvent(st, ctx->ev_pivot, 0);
+  EAR_TRY(s);
   EAR_CUDA_TRY(cudaGetLastError());
   return EAR_OK;
 }
 
-// Sharded FW on a rank's owned int32 rows: the 16-bit schedule first (allow16), the int32 one when it
-// did not apply.  lab / n_real as for fw_single.
-ear_status_t fw_sharded_auto(int32_t *S, int64_t ldd, int32_t Np, ear_comm_s *comm, const int32_t *lab,
-                             int32_t n_real, bool allow16, cudaStream_t st, ear_plan_s *plan) {
-  if (allow16 && Np >= 2 * TILE) {
-    Shard sh;
-    EAR_TRY(shard_setup(&sh, S, ldd, Np, comm->nranks, comm->rank, st));
-    std::vector<Shard *> v{&sh};
-    bool done = false;
-    ear_status_t s = fw_sharded16(v, Np, comm, lab, n_real, &done, st, false, plan);
-    shard_free(&sh, st);
-    EAR_TRY(s);
-    prof_fw16(done);
-    if (done) return EAR_OK;
-  }
-  return fw_sharded(S, ldd, Np, comm, st);
-}
+std::vector<int32_t> shard_rows(int32_t nt, int32_t P, int32_t rank) { return shard_rows_of(nt, P, rank); }
 
-// One rank's device work of a P-rank packed sharded FW, without the other ranks and the exchange
-// (apsp_reduced_rank_timing: per-rank compute scaling measured on one GPU).
-ear_status_t fw_rank_timing(const ear_plan_s *plan, int32_t Np, int32_t P, int32_t rank, cudaStream_t st) {
-  const size_t nown = shard_rows(Np / TILE, P, rank).size();
-  int32_t *S = nullptr;
-  EAR_CUDA_TRY(cudaMallocAsync((void **)&S, sizeof(int32_t) * std::max<size_t>(nown, 1) * TILE * Np, st));
-  Shard sh;
-  ear_status_t s = shard_setup(&sh, S, Np, Np, P, rank, st);
-  for (int32_t lr = 0; lr < sh.nown && s == EAR_OK; ++lr)
-    s = fw_init_D(plan, S + (int64_t)lr * TILE * Np, Np, Np, sh.rows[lr] * TILE, TILE, st);
-  bool done = false;
-  std::vector<Shard *> v{&sh};
-  if (s == EAR_OK) s = fw_sharded16(v, Np, nullptr, nullptr, plan->n_reduced, &done, st, true);
-  shard_free(&sh, st);
-  cudaFreeAsync(S, st);
-  return s;
-}
-
-// Full D from every rank's owned upper tiles (INF fill + scatter + all-reduce MIN).
-ear_status_t fw_sharded_gather(const int32_t *S, int64_t ldd, int32_t Np, int32_t *Df, int64_t ldf, ear_comm_s *comm,
-                               cudaStream_t st) {
-  Shard sh;
-  EAR_TRY(shard_setup(&sh, const_cast<int32_t *>(S), ldd, Np, comm->nranks, comm->rank, st));
-  ear_status_t status = EAR_OK;
-  if (ldf == Np) {
-    status = fill(Df, (int64_t)Np * Np, INF, st);
-  } else {
-    for (int32_t r = 0; r < Np && status == EAR_OK; ++r) status = fill(Df + (int64_t)r * ldf, Np, INF, st);
-  }
-  if (status == EAR_OK && sh.nown > 0) {
-    dim3 g(16, sh.nt, sh.nown);
-    EAR_LAUNCH(k_scatter_upper, g, 256, 0, st)(sh.S, sh.ldd, sh.d_rows, Df, ldf);
-  }
-  if (status == EAR_OK) {
-    int sc = prof_begin(PK_COMM, st);
-    if (ldf == Np) {
-      status = comm_allreduce_min(comm, Df, (int64_t)Np * Np, st);
-    } else {
-      for (int32_t r = 0; r < Np && status == EAR_OK; ++r) status = comm_allreduce_min(comm, Df + (int64_t)r * ldf, Np, st);
-    }
-    prof_end(sc, st, 0);
-  }
-  shard_free(&sh, st);
-  if (status != EAR_OK) return status;
-  EAR_CUDA_TRY(cudaGetLastError());
-  return EAR_OK;
-}
-
-int32_t shard_nown(int32_t nt, int32_t P, int32_t rank) { return (int32_t)shard_rows(nt, P, rank).size(); }
+int32_t shard_nown(int32_t nt, int32_t P, int32_t rank) { return (int32_t)shard_rows_of(nt, P, rank).size(); }
 
 ear_status_t shard_rows_device(int32_t nt, int32_t P, int32_t rank, int32_t **d_rows, int32_t *nown, cudaStream_t st) {
-  std::vector<int32_t> rows = shard_rows(nt, P, rank);
+  std::vector<int32_t> rows = shard_rows_of(nt, P, rank);
   *nown = (int32_t)rows.size();
   EAR_CUDA_TRY(cudaMallocAsync((void **)d_rows, sizeof(int32_t) * std::max<size_t>(rows.size(), 1), st));
   if (!rows.empty()) {
@@ -2021,56 +1600,99 @@ ear_status_t shard_rows_device(int32_t nt, int32_t P, int32_t rank, int32_t **d_
   return EAR_OK;
 }
 
+// this rank's owned-row storage inside its window (collective: reserves the window for Np)
+ear_status_t fw_shard_buffer(ear_comm_s *comm, int32_t Np, cudaStream_t st, int32_t **S) {
+  const int32_t nown = shard_nown(Np / TILE, comm->nranks, comm->rank);
+  EAR_TRY(comm_reserve(comm, Np, nown, st));
+  *S = comm_region(comm, comm->rank);
+  return EAR_OK;
+}
+
+// Sharded FW on a rank's owned int32 rows S (ld ldd >= Np): packed schedule first (allow16), int32
+// otherwise.  Collective over the communicator's ranks.
+ear_status_t fw_sharded_auto(int32_t *S, int64_t ldd, int32_t Np, ear_comm_s *comm, const int32_t *lab,
+                             int32_t n_real, bool allow16, cudaStream_t st, ear_plan_s *plan) {
+  EAR_TRY(comm_reserve(comm, Np, shard_nown(Np / TILE, comm->nranks, comm->rank), st));
+  Scratch sc(st);
+  Shard sh;
+  EAR_TRY(shard_setup(&sh, S, ldd, Np, comm->nranks, comm->rank, sc));
+  std::vector<Shard *> v{&sh};
+  bool used16 = false;
+  EAR_TRY(fw_sharded_run(v, Np, comm, lab, n_real, allow16, st, plan, false, &used16));
+  if (allow16 && Np >= 2 * TILE) prof_fw16(used16);
+  EAR_CUDA_TRY(cudaGetLastError());
+  return EAR_OK;
+}
+
+// One rank's device work of a P-rank sharded FW, without the other ranks and the exchange
+// (apsp_reduced_rank_timing: per-rank compute scaling measured on one GPU); packed unless fw32.
+ear_status_t fw_rank_timing(const ear_plan_s *plan, int32_t Np, int32_t P, int32_t rank, bool fw32, cudaStream_t st) {
+  Scratch sc(st);
+  const size_t nown = shard_rows_of(Np / TILE, P, rank).size();
+  int32_t *S = nullptr;
+  if (!sc.get(&S, std::max<size_t>(nown, 1) * TILE * Np)) { set_error("rank timing: out of memory"); return EAR_ENOMEM; }
+  Shard sh;
+  EAR_TRY(shard_setup(&sh, S, Np, Np, P, rank, sc));
+  for (int32_t lr = 0; lr < sh.nown; ++lr)
+    EAR_TRY(fw_init_D(plan, S + (int64_t)lr * TILE * Np, Np, Np, sh.rows[lr] * TILE, TILE, st));
+  std::vector<Shard *> v{&sh};
+  bool used16 = false;
+  return fw_sharded_run(v, Np, nullptr, nullptr, plan->n_reduced, !fw32, st, nullptr, true, &used16);
+}
+
+// Full D (Np x Np, ldf) from every rank's owned upper tiles: the rank's storage S goes into its window
+// region (unless it is already there), a barrier, then every rank reads every tile from the window of
+// its owner (the mirror of the lower triangle fused into the same pass), then a barrier so no rank
+// rewrites its region while a peer still reads it.  Collective.
+ear_status_t fw_sharded_gather(const int32_t *S, int64_t ldd, int32_t Np, int32_t *Df, int64_t ldf, ear_comm_s *comm,
+                               cudaStream_t st) {
+  const int32_t nt = Np / TILE, P = comm->nranks;
+  const int32_t nown = shard_nown(nt, P, comm->rank);
+  EAR_TRY(comm_reserve(comm, Np, nown, st));
+  int32_t *reg = comm_region(comm, comm->rank);
+  if (S != reg && nown > 0)
+    EAR_CUDA_TRY(cudaMemcpy2DAsync(reg, sizeof(int32_t) * Np, S, sizeof(int32_t) * ldd, sizeof(int32_t) * Np,
+                                   (size_t)nown * TILE, cudaMemcpyDeviceToDevice, st));
+  int sc = prof_begin(PK_COMM, st);
+  EAR_TRY(comm_barrier(comm, st));
+  PeerPtrs regions{};
+  regions.n = P;
+  for (int p = 0; p < P; ++p) regions.p[p] = reinterpret_cast<char *>(comm_region(comm, p));
+  if (nt > 0) EAR_LAUNCH(k_gather_pull, dim3(nt, nt), 256, 0, st)(regions, P, Np, Df, ldf);
+  EAR_TRY(comm_barrier(comm, st));
+  prof_end(sc, st, 0);
+  EAR_CUDA_TRY(cudaGetLastError());
+  return EAR_OK;
+}
+
 // The same schedule for P ranks emulated in one process on one device (tests of the multi-GPU path on
-// one GPU): every virtual rank has its own owned storage, the shared prow stands in for the
-// all-reduce (the ranks' pieces are disjoint), and the ranks' upper tiles are scattered into D.
-ear_status_t fw_sharded_emulated(ear_plan_s *plan, int32_t *D, int64_t ldd, int32_t Np, int32_t P,
-                                 cudaStream_t st) {
+// one GPU): every virtual rank has its own owned storage, they share the pivot-row buffers (their pieces
+// are disjoint), and the ranks' upper tiles are scattered into D.
+ear_status_t fw_sharded_emulated(ear_plan_s *plan, int32_t *D, int64_t ldd, int32_t Np, int32_t P, cudaStream_t st) {
   const int nt = Np / TILE;
+  Scratch sc(st);
   std::vector<Shard> sh(P);
-  ear_status_t status = EAR_OK;
-  for (int r = 0; r < P && status == EAR_OK; ++r) {
-    const size_t nown = shard_rows(nt, P, r).size();
+  for (int r = 0; r < P; ++r) {
+    const size_t nown = shard_rows_of(nt, P, r).size();
     int32_t *S = nullptr;
-    EAR_CUDA_TRY(cudaMallocAsync((void **)&S, sizeof(int32_t) * std::max<size_t>(nown, 1) * TILE * Np, st));
-    status = shard_setup(&sh[r], S, Np, Np, P, r, st);
-    for (int32_t lr = 0; lr < sh[r].nown && status == EAR_OK; ++lr)
-      status = fw_init_D(plan, S + (int64_t)lr * TILE * Np, Np, Np, sh[r].rows[lr] * TILE, TILE, st);
+    if (!sc.get(&S, std::max<size_t>(nown, 1) * TILE * Np)) { set_error("emulated: out of memory"); return EAR_ENOMEM; }
+    EAR_TRY(shard_setup(&sh[r], S, Np, Np, P, r, sc));
+    for (int32_t lr = 0; lr < sh[r].nown; ++lr)
+      EAR_TRY(fw_init_D(plan, S + (int64_t)lr * TILE * Np, Np, Np, sh[r].rows[lr] * TILE, TILE, st));
   }
-  bool done16 = false;
-  if (status == EAR_OK && !(plan->flags & EAR_FLAG_FW32) && Np >= 2 * TILE) {
-    const int32_t *lab = nullptr;
-    status = reduced_labels(plan, Np, st, &lab);
-    std::vector<Shard *> v;
-    for (int r = 0; r < P; ++r) v.push_back(&sh[r]);
-    if (status == EAR_OK) status = fw_sharded16(v, Np, nullptr, lab, plan->n_reduced, &done16, st, false, plan);
-    if (status == EAR_OK) prof_fw16(done16);
-  }
-  int32_t *prow = nullptr;
-  if (status == EAR_OK && !done16) {
-    cudaError_t e = cudaMallocAsync((void **)&prow, sizeof(int32_t) * (size_t)TILE * Np, st);
-    if (e != cudaSuccess) { set_error("emulated prow: %s", cudaGetErrorString(e)); status = EAR_ENOMEM; }
-  }
-  CUtensorMap map_prow;
-  if (status == EAR_OK && !done16) status = make_map(&map_prow, prow, TILE, Np, Np, fw_kc());
-  for (int k = 0; k < nt && status == EAR_OK && !done16; ++k) {
-    status = fill(prow, (int64_t)TILE * Np, INF, st);
-    for (int r = 0; r < P && status == EAR_OK; ++r) status = shard_xfer(sh[r], k, prow, 0, st);
-    if (status == EAR_OK) status = shard_pivot(prow, map_prow, Np, k, st);
-    for (int r = 0; r < P && status == EAR_OK; ++r) status = shard_xfer(sh[r], k, prow, 1, st);
-    for (int r = 0; r < P && status == EAR_OK; ++r) status = shard_phase3(sh[r], map_prow, k, st);
-  }
-  for (int r = 0; r < P && status == EAR_OK; ++r) {
+  const bool allow16 = !(plan->flags & EAR_FLAG_FW32);
+  const int32_t *lab = nullptr;
+  if (allow16) EAR_TRY(reduced_labels(plan, Np, st, &lab));
+  std::vector<Shard *> v;
+  for (int r = 0; r < P; ++r) v.push_back(&sh[r]);
+  bool used16 = false;
+  EAR_TRY(fw_sharded_run(v, Np, nullptr, lab, plan->n_reduced, allow16, st, plan, false, &used16));
+  if (allow16 && Np >= 2 * TILE) prof_fw16(used16);
+  for (int r = 0; r < P; ++r) {
     if (sh[r].nown == 0) continue;
     dim3 g(16, nt, sh[r].nown);
     EAR_LAUNCH(k_scatter_upper, g, 256, 0, st)(sh[r].S, sh[r].ldd, sh[r].d_rows, D, ldd);
   }
-  if (prow) cudaFreeAsync(prow, st);
-  for (int r = 0; r < P; ++r) {
-    if (sh[r].S) cudaFreeAsync(sh[r].S, st);
-    shard_free(&sh[r], st);
-  }
-  if (status != EAR_OK) return status;
   EAR_CUDA_TRY(cudaGetLastError());
   return EAR_OK;
 }
@@ -2090,8 +1712,8 @@ ear_status_t reduced_labels(ear_plan_s *p, int32_t Np, cudaStream_t st, const in
       int32_t h = 0;
       if (p->n_redges == 0) break;
       dev_memset(changed, 0, sizeof(int32_t), st);
-      EAR_LAUNCH(k_cc_hook16, grid_for(p->n_redges), 256, 0, st)(p->re_u, p->re_v, p->n_redges, p->cc, changed);
-      EAR_LAUNCH(k_cc_jump16, grid_for(Np), 256, 0, st)(p->cc, Np);
+      EAR_LAUNCH(k_cc_hook, grid_for(p->n_redges), 256, 0, st)(p->re_u, p->re_v, p->n_redges, p->cc, changed);
+      EAR_LAUNCH(k_cc_jump, grid_for(Np), 256, 0, st)(p->cc, Np);
       Readback rb(st);
       cudaError_t e = rb.get(&h, changed, sizeof(int32_t));
       if (e == cudaSuccess) e = rb.sync();

@@ -176,6 +176,39 @@ cudaError_t readback_direct(void *h_mapped, const void *d_src, size_t bytes, cud
   return bytes ? launch_readback(h_mapped, d_src, bytes, st) : cudaSuccess;
 }
 
+// ---- per-device helpers
+int num_sms() {
+  static std::atomic<int> cache[64];
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return 148;
+  int v = cache[dev].load(std::memory_order_relaxed);
+  if (v) return v;
+  if (cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess || v < 1) v = 148;
+  cache[dev].store(v, std::memory_order_relaxed);
+  return v;
+}
+
+// cudaFuncSetAttribute(MaxDynamicSharedMemorySize) is per device and per kernel: raise it to the
+// largest size requested so far for (device, kernel), under a lock
+cudaError_t smem_attr(const void *kernel, int bytes) {
+  static std::mutex mu;
+  static std::vector<std::pair<std::pair<int, const void *>, int>> done;
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return e;
+  std::lock_guard<std::mutex> lk(mu);
+  for (auto &d : done)
+    if (d.first.first == dev && d.first.second == kernel) {
+      if (d.second >= bytes) return cudaSuccess;
+      e = cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
+      if (e == cudaSuccess) d.second = bytes;
+      return e;
+    }
+  e = cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
+  if (e == cudaSuccess) done.push_back({{dev, kernel}, bytes});
+  return e;
+}
+
 }  // namespace ear
 
 using namespace ear;

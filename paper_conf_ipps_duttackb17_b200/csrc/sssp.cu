@@ -470,11 +470,7 @@ template <int NTS, int K>
 static ear_status_t sssp_launch(ear_plan_s *p, int32_t *D, int64_t ldd, int32_t Np, int32_t row0, int32_t rows,
                                 const int32_t *trows,
                                 int smem_s, int nsm, unsigned long long *d_stats, cudaStream_t st) {
-  static int attr_s = 0;
-  if (smem_s > attr_s) {
-    EAR_CUDA_TRY(cudaFuncSetAttribute(k_sssp_smem<NTS, K>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_s));
-    attr_s = smem_s;
-  }
+  EAR_CUDA_TRY(smem_attr((const void *)k_sssp_smem<NTS, K>, smem_s));
   int per_sm = 1;
   EAR_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_sssp_smem<NTS, K>, NTS, smem_s));
   const int64_t grid = std::min<int64_t>(rows, (int64_t)nsm * std::max(per_sm, 1));
@@ -502,11 +498,7 @@ static ear_status_t sssp_list_launch(ear_plan_s *p, int32_t *D, int64_t ldd, int
   const int fixed = 4 * Np + 8 * W + 64;
   const int cap = std::min(Np, (max_smem - fixed) / 8);
   const int smem = 4 * Np + 8 * cap + 8 * W;
-  static int attr = 0;
-  if (smem > attr) {
-    EAR_CUDA_TRY(cudaFuncSetAttribute(k_sssp_list<NTS, K>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
-    attr = smem;
-  }
+  EAR_CUDA_TRY(smem_attr((const void *)k_sssp_list<NTS, K>, smem));
   int per_sm = 1;
   EAR_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_sssp_list<NTS, K>, NTS, smem));
   const int64_t grid = std::min<int64_t>(rows, (int64_t)nsm * std::max(per_sm, 1));
@@ -590,11 +582,7 @@ ear_status_t sssp_rows(ear_plan_s *p, int32_t *D, int64_t ldd, int32_t Np, int32
     }
   }
   const int smem = 2 * W * 4;
-  static int attr = 0;
-  if (smem > attr) {
-    EAR_CUDA_TRY(cudaFuncSetAttribute(k_sssp_bf, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
-    attr = smem;
-  }
+  EAR_CUDA_TRY(smem_attr((const void *)k_sssp_bf, smem));
   int per_sm = 1;
   EAR_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_sssp_bf, NT, smem));
   // concurrent rows live in L2: cap the number of resident sources (rows of 4*Np bytes) near 96 MB

@@ -88,8 +88,7 @@ SIGNATURES = {
     "apsp_full_host_async": (_I32, [_I32, _I64, _P, _P, _P, _U32, _I32, _I32, _P, _I64, _P, _P, ctypes.POINTER(_P)]),
     "ear_job_wait": (_I32, [_P]),
     "ear_row_block": (None, [_I32, _I32, _I32, ctypes.POINTER(_I32), ctypes.POINTER(_I32)]),
-    "ear_comm_unique_id": (_I32, [ctypes.c_char_p]),
-    "ear_comm_init": (_I32, [ctypes.c_char_p, _I32, _I32, ctypes.POINTER(_P)]),
+    "ear_comm_init": (_I32, [_I32, _I32, _P, _P, ctypes.POINTER(_P)]),
     "ear_comm_info": (_I32, [_P, ctypes.POINTER(_I32), ctypes.POINTER(_I32)]),
     "ear_comm_destroy": (None, [_P]),
     "ear_profile_enable": (None, [_I32]),
@@ -134,6 +133,15 @@ def _stream(stream=None) -> int:
     return stream.cuda_stream
 
 
+def _check_out(out: torch.Tensor, rows: int, n: int, cuda: bool):
+    """`out` must hold rows x n int32 entries with unit column stride (the library writes every one)."""
+    where = "CUDA" if cuda else "host"
+    if out.is_cuda != cuda or out.dtype != torch.int32 or out.dim() != 2 or out.stride(1) != 1:
+        raise EarError(f"out must be a 2-D int32 {where} tensor with unit column stride")
+    if out.shape[0] < rows or out.shape[1] < n or out.stride(0) < n:
+        raise EarError(f"out is {tuple(out.shape)} (row stride {out.stride(0)}); need at least {rows} x {n}")
+
+
 def _dev_i32(t: torch.Tensor, name: str) -> torch.Tensor:
     if not (t.is_cuda and t.dtype == torch.int32 and t.is_contiguous()):
         raise EarError(f"{name} must be a contiguous int32 CUDA tensor")
@@ -154,32 +162,47 @@ class PlanInfo:
     max_weight: int
 
 
+# int32_t (*ear_allgather_fn)(const void *send, void *recv, int64_t bytes, void *ctx)
+ALLGATHER_FN = ctypes.CFUNCTYPE(ctypes.c_int32, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_int64, ctypes.c_void_p)
+
+
 class Comm:
-    """NCCL communicator of this rank (one process per GPU), created collectively.  The unique id is
-    made on rank 0 by the library and distributed with torch.distributed."""
+    """This rank's communicator (one process per GPU; several processes may share a GPU): the
+    library's peer-memory exchange windows.  The library trades CUDA IPC handles through a host
+    all-gather callback, implemented here with torch.distributed (any backend; gloo works for ranks
+    that share a GPU)."""
 
-    def __init__(self, handle, nranks: int, rank: int):
-        self.handle, self.nranks, self.rank = handle, nranks, rank
-
-    @staticmethod
-    def distribute_unique_id(group=None) -> bytes:
-        """Rank 0 creates the NCCL unique id (library call); torch.distributed broadcasts it."""
-        import torch.distributed as dist
-        buf = ctypes.create_string_buffer(128)
-        if dist.get_rank(group) == 0:
-            _check(lib().ear_comm_unique_id(buf), "ear_comm_unique_id")
-        obj = [bytes(buf.raw)]
-        dist.broadcast_object_list(obj, src=0, group=group)
-        return obj[0]
+    def __init__(self, handle, nranks: int, rank: int, keep=None):
+        self.handle, self.nranks, self.rank, self._keep = handle, nranks, rank, keep
 
     @classmethod
     def from_torch_distributed(cls, group=None) -> "Comm":
         import torch.distributed as dist
         rank, world = dist.get_rank(group), dist.get_world_size(group)
-        uid = cls.distribute_unique_id(group)
+
+        def allgather(send, recv, nbytes, _ctx):
+            try:
+                out = [None] * world
+                dist.all_gather_object(out, ctypes.string_at(send, nbytes), group=group)
+                buf = b"".join(out)
+                if len(buf) != nbytes * world:
+                    return 1
+                ctypes.memmove(recv, buf, len(buf))
+                return 0
+            except Exception:  # noqa: BLE001  (reported to the library as a failed collective)
+                return 1
+
+        fn = ALLGATHER_FN(allgather)
         h = _P()
-        _check(lib().ear_comm_init(uid, world, rank, ctypes.byref(h)), "ear_comm_init")
-        return cls(h, world, rank)
+        _check(lib().ear_comm_init(world, rank, ctypes.cast(fn, _P), None, ctypes.byref(h)), "ear_comm_init")
+        return cls(h, world, rank, keep=fn)
+
+    @classmethod
+    def single(cls) -> "Comm":
+        """A one-rank communicator (the sharded code path on one process, no peers)."""
+        h = _P()
+        _check(lib().ear_comm_init(1, 0, None, None, ctypes.byref(h)), "ear_comm_init")
+        return cls(h, 1, 0)
 
     def destroy(self):
         if self.handle:
@@ -292,8 +315,7 @@ def expand_ears(plan: Plan, D_full: torch.Tensor, row_begin: int, row_end: int, 
     if out is None:
         out = torch.empty((row_end - row_begin, plan.n), dtype=torch.int32, device="cuda")
     _dev_i32(D_full, "D_full")
-    if not (out.is_cuda and out.dtype == torch.int32 and out.stride(1) == 1):
-        raise EarError("out must be an int32 CUDA tensor with unit column stride")
+    _check_out(out, row_end - row_begin, plan.n, cuda=True)
     _check(lib().expand_ears(plan.handle, D_full.data_ptr(), D_full.stride(0), row_begin, row_end, out.data_ptr(),
                              out.stride(0), _stream(stream)), "expand_ears")
     return out
@@ -303,8 +325,13 @@ def query_pairs(plan: Plan, D_full: torch.Tensor, s: torch.Tensor, t: torch.Tens
                 out: torch.Tensor | None = None, stream=None) -> torch.Tensor:
     """Compact/query mode: S[s[i], t[i]] from D and the plan's descriptors (no N x N matrix)."""
     s, t = _dev_i32(s, "s"), _dev_i32(t, "t")
+    if t.numel() != s.numel():
+        raise EarError(f"s and t differ in length ({s.numel()} vs {t.numel()})")
     if out is None:
         out = torch.empty(s.numel(), dtype=torch.int32, device="cuda")
+    _dev_i32(out, "out")
+    if out.numel() < s.numel():
+        raise EarError(f"out holds {out.numel()} entries for {s.numel()} pairs")
     _check(lib().ear_query_pairs(plan.handle, _dev_i32(D_full, "D_full").data_ptr(), D_full.stride(0), s.numel(),
                                  s.data_ptr(), t.data_ptr(), out.data_ptr(), _stream(stream)), "ear_query_pairs")
     return out
@@ -324,6 +351,7 @@ def apsp_full(n: int, src: torch.Tensor, dst: torch.Tensor, w: torch.Tensor, out
     src, dst, w = _dev_i32(src, "src"), _dev_i32(dst, "dst"), _dev_i32(w, "w")
     if out is None:
         out = torch.empty((row_end - row_begin, n), dtype=torch.int32, device="cuda")
+    _check_out(out, row_end - row_begin, n, cuda=True)
     _check(lib().apsp_full(n, src.numel(), src.data_ptr(), dst.data_ptr(), w.data_ptr(), flags, row_begin, row_end,
                            out.data_ptr(), out.stride(0), _comm_handle(comm), _stream(stream)), "apsp_full")
     return out
@@ -341,8 +369,7 @@ def apsp_full_host(n: int, src: np.ndarray | torch.Tensor, dst, w, out: torch.Te
             raise EarError("apsp_full_host takes contiguous int32 host arrays")
     if out is None:
         out = torch.empty((row_end - row_begin, n), dtype=torch.int32, pin_memory=True)
-    if out.is_cuda or out.dtype != torch.int32 or out.stride(1) != 1:
-        raise EarError("out must be a host int32 tensor with unit column stride")
+    _check_out(out, row_end - row_begin, n, cuda=False)
     _check(lib().apsp_full_host(n, tens[0].numel(), tens[0].data_ptr(), tens[1].data_ptr(), tens[2].data_ptr(),
                                 flags, row_begin, row_end, out.data_ptr(), out.stride(0), _comm_handle(comm),
                                 _stream(stream)), "apsp_full_host")
@@ -361,6 +388,14 @@ class HostJob:
             _check(lib().ear_job_wait(h), "ear_job_wait")
         return self.out
 
+    def __del__(self):  # pragma: no cover
+        # a job dropped without wait() still owns device scratch and writes into `out`: finish it
+        # before `out` (possibly torch's cached pinned memory) can be handed to anyone else
+        try:
+            self.wait()
+        except Exception:
+            pass
+
 
 def apsp_full_host_async(n: int, src, dst, w, out: torch.Tensor | None = None, row_begin: int = 0,
                          row_end: int | None = None, flags: int = 0, comm: Comm | None = None,
@@ -376,8 +411,7 @@ def apsp_full_host_async(n: int, src, dst, w, out: torch.Tensor | None = None, r
             raise EarError("apsp_full_host_async takes contiguous int32 host arrays")
     if out is None:
         out = torch.empty((row_end - row_begin, n), dtype=torch.int32, pin_memory=True)
-    if out.is_cuda or out.dtype != torch.int32 or out.stride(1) != 1:
-        raise EarError("out must be a host int32 tensor with unit column stride")
+    _check_out(out, row_end - row_begin, n, cuda=False)
     h = ctypes.c_void_p()
     _check(lib().apsp_full_host_async(n, tens[0].numel(), tens[0].data_ptr(), tens[1].data_ptr(), tens[2].data_ptr(),
                                       flags, row_begin, row_end, out.data_ptr(), out.stride(0), _comm_handle(comm),

@@ -234,6 +234,72 @@ def test_certificate_catches_perturbations():
         assert not pins.bellman_certificate(P, rows, g.n, g.src, g.dst, g.w)
 
 
+# ------------------------------------------------------------------------------ P4, the C checker
+# oracle.certify_rows (oracle/apsp_oracle.c) is what certifies the full cfg4 / cfg5 matrices
+# (tests/test_full_verify_gpu.py).  Pinned here: it accepts the oracle's rows, it agrees with the numpy
+# certificate on perturbed rows, and -- exhaustively on small graphs -- the true row is the ONLY row it
+# accepts (uniqueness of the Bellman fixed point with weights >= 1).
+@pytest.mark.parametrize("seed", range(12))
+def test_c_certificate_accepts_oracle_rows(seed):
+    g = gg.corner_cases(seed, n_target=30 + 40 * seed)
+    S = oracle.apsp(g.n, g.src, g.dst, g.w)
+    assert oracle.certify_rows(g.n, g.src, g.dst, g.w, np.arange(g.n), S) == (0, None)
+
+
+def test_c_certificate_accepts_cfg_rows():
+    for name, rows in (("cfg1", np.arange(2000)), ("cfg2", np.arange(0, 20000, 97))):
+        g = gg.config(name)
+        S = oracle.apsp_rows(g.n, g.src, g.dst, g.w, rows)
+        assert oracle.certify_rows(g.n, g.src, g.dst, g.w, rows, S) == (0, None)
+
+
+def test_c_certificate_agrees_with_numpy_on_perturbations():
+    g = gg.corner_cases(7, n_target=50)
+    S = oracle.apsp(g.n, g.src, g.dst, g.w)
+    rows = np.arange(g.n)
+    rng = np.random.default_rng(3)
+    for trial in range(200):
+        P = S.copy()
+        s, t = (int(x) for x in rng.integers(0, g.n, 2))
+        kind = trial % 4
+        if kind == 0:
+            P[s, t] += 1 if P[s, t] < INF else -1
+        elif kind == 1:
+            P[s, t] = P[s, t] - 1 if P[s, t] > 0 else 1
+        elif kind == 2:
+            P[s, t] = INF if P[s, t] != INF else 0
+        else:   # swap two different entries of a row
+            u = (t + 1 + int(rng.integers(0, g.n - 1))) % g.n
+            if P[s, t] == P[s, u]:
+                continue
+            P[s, t], P[s, u] = P[s, u], P[s, t]
+        bad, first = oracle.certify_rows(g.n, g.src, g.dst, g.w, rows, P)
+        assert bad > 0 and first[0] == s
+        assert not pins.bellman_certificate(P, rows, g.n, g.src, g.dst, g.w)
+
+
+def test_c_certificate_unique_fixed_point_exhaustive_n4():
+    # every graph on 4 labelled vertices, each edge absent or weight 1 or 2 (3^6 = 729 graphs); for every
+    # source, all 8^4 candidate rows over {0..6, INF}: exactly one is accepted, the brute-force FW row
+    n = 4
+    vals = np.array(list(range(7)) + [INF], dtype=np.int32)
+    cand = np.array(list(itertools.product(vals, repeat=n)), dtype=np.int32)   # (4096, 4)
+    pairs = list(itertools.combinations(range(n), 2))
+    graphs = 0
+    for assign in itertools.product((0, 1, 2), repeat=len(pairs)):
+        edges = [(a, b, x) for (a, b), x in zip(pairs, assign) if x]
+        src = np.array([e[0] for e in edges], np.int32)
+        dst = np.array([e[1] for e in edges], np.int32)
+        w = np.array([e[2] for e in edges], np.int32)
+        truth = pins.brute_fw(n, src, dst, w)
+        for s in range(n):
+            _, _, per = oracle.certify_rows(n, src, dst, w, np.full(len(cand), s), cand, per_row=True)
+            ok = np.flatnonzero(per == 0)
+            assert len(ok) == 1 and np.array_equal(cand[ok[0]], truth[s]), (edges, s)
+        graphs += 1
+    assert graphs == 3 ** 6
+
+
 # ------------------------------------------------------------------------------ P5 library routine
 @pytest.mark.parametrize("name,nrows", [("cfg1", None), ("cfg2", 200), ("cfg4", 24)])
 def test_oracle_matches_scipy(name, nrows):
