@@ -79,3 +79,14 @@ def test_product_package_never_imports_the_oracle():
             if f.endswith((".py", ".cu", ".cuh", ".h")):
                 src = open(os.path.join(dirpath, f)).read()
                 assert "import oracle" not in src and "from oracle" not in src and "apsp_oracle" not in src, f
+
+
+def test_only_test_infrastructure_uses_the_oracle():
+    """oracle/ is test infrastructure: only tests/, bench.py (cpu_baseline / reference arm) and
+    __graft_entry__.smoke() may import it -- not the package, tools/ or microbench/."""
+    for sub in ("paper_conf_ipps_duttackb17_b200", "tools", "microbench"):
+        for dirpath, _, files in os.walk(os.path.join(ROOT, sub)):
+            for f in files:
+                if f.endswith((".py", ".cu", ".cuh", ".h", ".sh")):
+                    src = open(os.path.join(dirpath, f)).read()
+                    assert not re.search(r"^\s*(import oracle|from oracle)", src, flags=re.M), os.path.join(dirpath, f)

@@ -2,8 +2,8 @@
 """cfg5 (BASELINE.json configs[4]): the 200k-vertex power-grid-like graph, full N x N APSP (160 GB of
 int32) produced on ONE B200 by row blocks -- the same per-rank work an 8-GPU row-block run does,
 executed block after block: Phase I + Phase II once (D = 59,850^2 reduced distances, 14.3 GB), then
-the ear expansion of each 25,000-row block (20 GB) into one reused device buffer.  Sampled rows of
-every block are checked bit for bit against the CPU oracle (test infrastructure, bounded sample).
+the ear expansion of each 25,000-row block (20 GB) into one reused device buffer.  Timing only: the
+whole 160 GB matrix is certified against the oracle by tests/test_full_verify_gpu.py (EAR_VERIFY_CFG5=1).
 
 Prints one JSON line: per-phase device times, entries/s over the whole job, parity counts.
 """
@@ -26,11 +26,9 @@ def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--config", default="cfg5")
     ap.add_argument("--block", type=int, default=25000)
-    ap.add_argument("--check-rows", type=int, default=4, help="oracle-checked rows per block")
     ap.add_argument("--phase2", choices=["fw", "sssp", "bcc"], default="fw")
     ap.add_argument("--warmup", type=int, default=1, help="untimed Phase II runs before the timed one")
     args = ap.parse_args()
-    import oracle
 
     g = gg.config(args.config)
     src, dst, w = (torch.as_tensor(x).cuda() for x in (g.src, g.dst, g.w))
@@ -56,8 +54,6 @@ def main():
     torch.cuda.synchronize()
     ms_dec, ms_p2 = e0.elapsed_time(e1), e1.elapsed_time(e2)
     out = torch.empty((args.block, g.n), dtype=torch.int32, device="cuda")
-    rng = np.random.default_rng(5)
-    checked = mism = 0
     ms_exp = 0.0
     for b0 in range(0, g.n, args.block):
         b1 = min(g.n, b0 + args.block)
@@ -67,11 +63,6 @@ def main():
         b.record()
         torch.cuda.synchronize()
         ms_exp += a.elapsed_time(b)
-        rows = rng.choice(np.arange(b0, b1), args.check_rows, replace=False)
-        ref = oracle.apsp_rows(g.n, g.src, g.dst, g.w, rows)
-        got = out[torch.as_tensor(rows - b0).cuda().long()].cpu().numpy()
-        checked += got.size
-        mism += int(np.count_nonzero(got != ref))
     wall = time.perf_counter() - t_start
     total_ms = ms_dec + ms_p2 + ms_exp
     print(json.dumps({"config": args.config, "n": g.n, "m": g.m, "n_reduced": info.n_reduced,
@@ -80,7 +71,7 @@ def main():
                       "output_bytes": 4 * g.n * g.n, "D_bytes": 4 * info.n_reduced_padded ** 2,
                       "expand_GBps": 4.0 * g.n * g.n / (ms_exp / 1e3) / 1e9,
                       "fw_tminplus": (info.n_reduced_padded ** 3 / 2) / (ms_p2 / 1e3) / 1e12 if flags == 0 else None,
-                      "oracle_checked_entries": checked, "mismatches": mism, "wall_s_including_checks": wall}),
+                      "wall_s": wall}),
           flush=True)
 
 
