@@ -19,6 +19,11 @@ Functions (paper = /root/reference/PAPER.md, ``P:NN`` = line NN):
   Its only solution with integer weights >= 1 is S itself, and it costs O(N + M) per row, so it
   certifies whole N x N matrices (cfg4, cfg5) where Dijkstra from every source would take minutes.
 
+* :func:`mcb_horton` / :func:`mcb_depina` -- minimum cycle basis (paper sec. 3) of a
+  multigraph (self-loops and parallel edges allowed, as in G^r): Horton's algorithm [18] (the
+  Horton set + a GF(2) greedy) and de Pina's Algorithm 2 with the signed-graph search of sec. 3.2.1
+  (``mcb_oracle.c``).  Two independent routes to the unique MCB weight.
+
 Pinned by ``tests/test_oracle_pins.py``: brute-force Floyd-Warshall and exhaustive enumeration of
 all small graphs (P1), closed forms (P2), invariants (P3), the Bellman certificate (P4), scipy's
 Dijkstra (P5) and the paper's own identities / Fig. 4 chains (P6).
@@ -35,15 +40,16 @@ import numpy as np
 INF = 0x3FFFFFFF
 _HERE = os.path.dirname(os.path.abspath(__file__))
 _SRC = os.path.join(_HERE, "apsp_oracle.c")
+_SRCS = [_SRC, os.path.join(_HERE, "mcb_oracle.c")]
 _LIB = os.path.join(_HERE, "liboracle.so")
 _lib = None
 
 
 def build(force: bool = False) -> str:
     """Compile ``liboracle.so`` with gcc (plain C + OpenMP)."""
-    if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
+    if force or not os.path.exists(_LIB) or any(os.path.getmtime(_LIB) < os.path.getmtime(s) for s in _SRCS):
         tmp = _LIB + f".tmp{os.getpid()}"
-        subprocess.check_call(["gcc", "-O2", "-fopenmp", "-shared", "-fPIC", "-o", tmp, _SRC])
+        subprocess.check_call(["gcc", "-O2", "-fopenmp", "-shared", "-fPIC", "-o", tmp, *_SRCS])
         os.replace(tmp, _LIB)
     return _LIB
 
@@ -64,6 +70,10 @@ def _load():
         lib.oracle_certify_rows.argtypes = [ctypes.c_int32, ctypes.c_int64, P, P, P, ctypes.c_int32, P, P,
                                             ctypes.c_int64, ctypes.c_int32, P, P]
         lib.oracle_certify_rows.restype = ctypes.c_int64
+        lib.oracle_mcb_horton.argtypes = [ctypes.c_int32, ctypes.c_int64, P, P, P, P, P, P, P, ctypes.c_int64]
+        lib.oracle_mcb_horton.restype = ctypes.c_int
+        lib.oracle_mcb_depina.argtypes = [ctypes.c_int32, ctypes.c_int64, P, P, P, P, P, P]
+        lib.oracle_mcb_depina.restype = ctypes.c_int
         _lib = lib
     return _lib
 
@@ -119,6 +129,38 @@ def certify_rows(n: int, src, dst, w, rows, D: np.ndarray, nthreads: int = 0, pe
         raise ValueError(f"oracle_certify_rows failed with status {bad}")
     res = (int(bad), (None if first[0] < 0 else (int(first[0]), int(first[1]))))
     return res + (rb,) if per_row else res
+
+
+def mcb_horton(n: int, src, dst, w):
+    """MCB by Horton's algorithm: ``(weight, dim, cycles)`` with every kept cycle as an int32 array of
+    edge indices (into src/dst/w), in the order the greedy kept them (non-decreasing weight)."""
+    src, dst, w = _edges(src, dst, w)
+    m = len(src)
+    weight = np.zeros(1, np.int64)
+    dim = np.zeros(1, np.int32)
+    off = np.zeros(m + 2, np.int64)
+    cap = max(1, 2 * (m + 1) * (n + 1))
+    cap = min(cap, 1 << 26)
+    edges = np.zeros(cap, np.int32)
+    st = _load().oracle_mcb_horton(n, m, _ptr(src), _ptr(dst), _ptr(w), _ptr(weight), _ptr(dim), _ptr(off),
+                                   _ptr(edges), cap)
+    if st != 0:
+        raise ValueError(f"oracle_mcb_horton failed with status {st}")
+    f = int(dim[0])
+    return int(weight[0]), f, [edges[off[i]:off[i + 1]].copy() for i in range(f)]
+
+
+def mcb_depina(n: int, src, dst, w):
+    """MCB by de Pina's Algorithm 2 (signed-graph search): ``(weight, dim, phase_weights)``."""
+    src, dst, w = _edges(src, dst, w)
+    m = len(src)
+    weight = np.zeros(1, np.int64)
+    dim = np.zeros(1, np.int32)
+    wts = np.zeros(max(m, 1), np.int64)
+    st = _load().oracle_mcb_depina(n, m, _ptr(src), _ptr(dst), _ptr(w), _ptr(weight), _ptr(dim), _ptr(wts))
+    if st != 0:
+        raise ValueError(f"oracle_mcb_depina failed with status {st}")
+    return int(weight[0]), int(dim[0]), wts[:int(dim[0])].copy()
 
 
 @dataclass

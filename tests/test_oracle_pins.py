@@ -408,3 +408,215 @@ def test_config_sizes_match_survey():
         g = gg.config(name)
         r = oracle.reduce_graph(g.n, g.src, g.dst, g.w)
         assert g.n == n and r.n_reduced == nr
+
+
+# ------------------------------------------------------------------------------ MCB oracle pins
+# (paper sec. 3).  oracle.mcb_horton (Horton [18]) and oracle.mcb_depina (Algorithm 2 with the
+# signed-graph search of sec. 3.2.1) are pinned against a brute force over the WHOLE cycle space of tiny
+# multigraphs, closed forms, and Lemma 3.1 (W(MCB(G)) = W(MCB(G^r)), equal dimensions).
+def _brute_mcb(n, src, dst, w):
+    """Enumerate all 2^f elements of the cycle space (xor of fundamental cycles of a BFS spanning
+    forest), keep the simple cycles (every vertex of degree 0 or 2, one connected piece), and run the
+    matroid greedy over them by weight."""
+    m = len(src)
+    adj = [[] for _ in range(n)]
+    for e in range(m):
+        adj[src[e]].append((dst[e], e))
+        adj[dst[e]].append((src[e], e))
+    par, pe, seen = [-1] * n, [-1] * n, [False] * n
+    intree = [False] * m
+    for r in range(n):
+        if seen[r]:
+            continue
+        seen[r] = True
+        q = [r]
+        for a in q:
+            for b, e in adj[a]:
+                if not seen[b]:
+                    seen[b] = True
+                    par[b], pe[b] = a, e
+                    intree[e] = True
+                    q.append(b)
+
+    def path_bits(a):
+        bits = 0
+        while par[a] >= 0:
+            bits ^= 1 << pe[a]
+            a = par[a]
+        return bits
+
+    fund = [path_bits(src[e]) ^ path_bits(dst[e]) ^ (1 << e) for e in range(m) if not intree[e]]
+    f = len(fund)
+    cycles = []
+    for mask in range(1, 1 << f):
+        v = 0
+        for i in range(f):
+            if mask >> i & 1:
+                v ^= fund[i]
+        es = [e for e in range(m) if v >> e & 1]
+        deg = [0] * n
+        for e in es:
+            deg[src[e]] += 1
+            deg[dst[e]] += 1
+        if any(d not in (0, 2) for d in deg):
+            continue
+        # connected: walk the edge set from one vertex
+        verts = {x for e in es for x in (src[e], dst[e])}
+        start = next(iter(verts))
+        reach, stack = {start}, [start]
+        while stack:
+            a = stack.pop()
+            for e in es:
+                for x, y in ((src[e], dst[e]), (dst[e], src[e])):
+                    if x == a and y not in reach:
+                        reach.add(y)
+                        stack.append(y)
+        if reach != verts:
+            continue
+        cycles.append((sum(w[e] for e in es), v))
+    cycles.sort(key=lambda c: c[0])
+    basis, total = {}, 0     # pivot bit -> vector (echelon form)
+    for wt, v in cycles:
+        while v:
+            p = v & -v
+            if p in basis:
+                v ^= basis[p]
+            else:
+                basis[p] = v
+                total += wt
+                break
+        if len(basis) == f:
+            break
+    assert len(basis) == f
+    return total, f
+
+
+def _rand_multigraph(rng):
+    n = int(rng.integers(2, 7))
+    m = int(rng.integers(n - 1, n + 6))
+    src, dst = [], []
+    for _ in range(m):
+        a = int(rng.integers(0, n))
+        b = a if rng.random() < 0.08 else int(rng.integers(0, n))   # some self-loops, many parallel edges
+        src.append(a)
+        dst.append(b)
+    w = [int(x) for x in rng.integers(1, 4, m)]                      # weights 1-3: many ties
+    return n, src, dst, w
+
+
+def test_mcb_oracles_match_brute_force_cycle_space():
+    rng = np.random.default_rng(11)
+    checked = 0
+    while checked < 250:
+        n, src, dst, w = _rand_multigraph(rng)
+        k = len({pins_find(n, src, dst, v) for v in range(n)})
+        if len(src) - n + k > 11:   # keep 2^f small
+            continue
+        bw, bf = _brute_mcb(n, src, dst, w)
+        hw, hf, cyc = oracle.mcb_horton(n, src, dst, w)
+        dw, df, _ = oracle.mcb_depina(n, src, dst, w)
+        assert (hw, hf) == (bw, bf) == (dw, df), (n, src, dst, w)
+        assert sum(int(sum(w[e] for e in c)) for c in cyc) == hw
+        checked += 1
+
+
+def pins_find(n, src, dst, v):
+    """component representative of v (union-find over the edge list)"""
+    p = list(range(n))
+
+    def f(x):
+        while p[x] != x:
+            x = p[x]
+        return x
+    for a, b in zip(src, dst):
+        ra, rb = f(a), f(b)
+        if ra != rb:
+            p[ra] = rb
+    return f(v)
+
+
+def _grid(gx, gy, s=0):
+    """gx x gy grid, every base edge subdivided by s unit-weight vertices (unit weights)"""
+    n = gx * gy
+    src, dst = [], []
+    for y in range(gy):
+        for x in range(gx):
+            i = y * gx + x
+            for j in ([i + 1] if x + 1 < gx else []) + ([i + gx] if y + 1 < gy else []):
+                prev = i
+                for _ in range(s):
+                    src.append(prev); dst.append(n); prev = n; n += 1
+                src.append(prev); dst.append(j)
+    return n, src, dst, [1] * len(src)
+
+
+@pytest.mark.parametrize("gx,gy,s", [(2, 2, 0), (3, 4, 0), (5, 5, 0), (4, 3, 2), (6, 2, 1)])
+def test_mcb_grid_closed_form(gx, gy, s):
+    # a grid's faces: (gx-1)(gy-1) cycles of weight 4(s+1) each, the girth -> MCB weight 4(s+1)(gx-1)(gy-1)
+    n, src, dst, w = _grid(gx, gy, s)
+    f = (gx - 1) * (gy - 1)
+    assert oracle.mcb_horton(n, src, dst, w)[:2] == (4 * (s + 1) * f, f)
+    if n <= 40:
+        assert oracle.mcb_depina(n, src, dst, w)[:2] == (4 * (s + 1) * f, f)
+
+
+@pytest.mark.parametrize("lens", [(1, 2, 3), (2, 2, 2), (1, 1, 5), (3, 4, 7)])
+def test_mcb_theta_closed_form(lens):
+    # two vertices joined by three paths of lengths a <= b <= c: MCB = {a+b, a+c}
+    a, b, c = sorted(lens)
+    n, src, dst = 2, [], []
+    for L in lens:
+        prev = 0
+        for _ in range(L - 1):
+            src.append(prev); dst.append(n); prev = n; n += 1
+        src.append(prev); dst.append(1)
+    w = [1] * len(src)
+    assert oracle.mcb_horton(n, src, dst, w)[:2] == (2 * a + b + c, 2)
+    assert oracle.mcb_depina(n, src, dst, w)[:2] == (2 * a + b + c, 2)
+
+
+@pytest.mark.parametrize("k", [3, 4, 5, 6])
+def test_mcb_complete_graph(k):
+    # K_k, unit weights: girth 3 and the triangles span the cycle space -> 3 * (m - n + 1)
+    src, dst = zip(*itertools.combinations(range(k), 2))
+    f = len(src) - k + 1
+    assert oracle.mcb_horton(k, src, dst, [1] * len(src))[:2] == (3 * f, f)
+    assert oracle.mcb_depina(k, src, dst, [1] * len(src))[:2] == (3 * f, f)
+
+
+@pytest.mark.parametrize("n", [3, 10, 57])
+def test_mcb_cycle_is_its_own_basis(n):
+    g = gg.cycle(n, seed=n)
+    assert oracle.mcb_horton(g.n, g.src, g.dst, g.w)[:2] == (int(g.w.sum()), 1)
+
+
+def _canonical(g):
+    """reading C3: drop self-loops, parallel edges -> the lightest"""
+    best = {}
+    for a, b, x in zip(g.src.tolist(), g.dst.tolist(), g.w.tolist()):
+        if a == b:
+            continue
+        key = (min(a, b), max(a, b))
+        best[key] = min(best.get(key, x), x)
+    ks = sorted(best)
+    return (np.array([k[0] for k in ks], np.int32), np.array([k[1] for k in ks], np.int32),
+            np.array([best[k] for k in ks], np.int32))
+
+
+@pytest.mark.parametrize("seed", range(15))
+def test_mcb_lemma_3_1_reduced_graph(seed):
+    # Lemma 3.1 (P:273-297): the MCB of G and of its reduced multigraph G^r (chains -> weighted edges,
+    # closed ears -> self-loops, parallel chains -> parallel edges) have the same weight and dimension
+    g = gg.corner_cases(seed, n_target=25 + 6 * seed)
+    s, d, w = _canonical(g)
+    red = oracle.reduce_graph(g.n, s, d, w)
+    terms = np.flatnonzero(red.term)
+    idx = -np.ones(g.n, np.int64)
+    idx[terms] = np.arange(len(terms))
+    ru, rv = idx[red.re_u], idx[red.re_v]
+    assert np.all(ru >= 0) and np.all(rv >= 0)
+    wg, fg, _ = oracle.mcb_horton(g.n, s, d, w)
+    wr, fr, _ = oracle.mcb_horton(len(terms), ru.astype(np.int32), rv.astype(np.int32), red.re_w.astype(np.int32))
+    assert (wg, fg) == (wr, fr)
+    if len(terms) <= 60 and fr <= 60:
+        assert oracle.mcb_depina(len(terms), ru.astype(np.int32), rv.astype(np.int32), red.re_w.astype(np.int32))[:2] == (wr, fr)
