@@ -174,6 +174,31 @@ def oracle_sample(g, target_s: float, rows_hint: int | None = None):
     return rows_hint * g.n / dt, rows_hint, dt, threads
 
 
+def host_info() -> dict:
+    """CPU model, nproc and the affinity count of this process."""
+    model = None
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                model = line.split(":", 1)[1].strip()
+                break
+    except OSError:
+        pass
+    return {"cpu_model": model, "nproc": os.cpu_count(), "affinity": len(os.sched_getaffinity(0))}
+
+
+def cfg1_one_core() -> dict:
+    """The oracle on ONE core over all of cfg1 (2,000 sources x 2,000 columns), SURVEY 8.d."""
+    import oracle
+    from paper_conf_ipps_duttackb17_b200 import graphgen as gg
+    g = gg.config("cfg1")
+    t = time.perf_counter()
+    oracle.apsp(g.n, g.src, g.dst, g.w, nthreads=1)
+    dt = time.perf_counter() - t
+    oracle.num_threads(len(os.sched_getaffinity(0)))   # back to every core this process may use
+    return {"seconds": dt, "entries_per_s": g.n * g.n / dt, "threads": 1}
+
+
 def run_reference(args, rank, world):
     """The reference arm for this tier: the CPU oracle, timed on the box's host cores."""
     if rank != 0:
@@ -205,7 +230,8 @@ def run_reference(args, rank, world):
             "data": "synthetic (seeded generator)",
             "config": {"workload": WORKLOADS.get(args.config, args.config), "name": args.config, "n": g.n,
                        "m": g.m, "seed": args.seed},
-            "cpu_baseline": {"value": value, "unit": UNIT, "cores": threads, "kind": "oracle", "sample": sample},
+            "cpu_baseline": dict({"value": value, "unit": UNIT, "cores": threads, "kind": "oracle", "sample": sample},
+                                 **host_info()),
             "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 
@@ -266,25 +292,40 @@ def run_ours(args, rank, world, local_rank):
     barrier()
     torch.cuda.synchronize()
 
+    # the headline: K steps with the library's per-launch profiling OFF (only its launch counter runs)
     sampler = ClockSampler(gpu_id_for(local_rank))
     sampler.start()
     time.sleep(0.3)
+    ea.profile_enable(False)
     ea.profile_reset()
-    ea.profile_enable(True)
-    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    ev0.record(stream)
-    for _ in range(args.steps):
+    evs = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps + 1)]
+    evs[0].record(stream)
+    for i in range(args.steps):
         step()
-    ev1.record(stream)
+        evs[i + 1].record(stream)
     torch.cuda.synchronize()
     barrier()
     torch.cuda.synchronize()
     clocks = sampler.stop()
-    prof = ea.profile_read()
-    ea.profile_enable(False)
-    ms = ev0.elapsed_time(ev1)
+    launches = int(ea.profile_read()["launches"])
+    ms = evs[0].elapsed_time(evs[-1])
+    step_ms = [evs[i].elapsed_time(evs[i + 1]) for i in range(args.steps)]
     ms_max = max_over_ranks(ms, world, dev)
     value = float(g.n) * float(g.n) * args.steps / (ms_max / 1e3)
+
+    # a separate profiled pass of the same K steps: CUDA events around every library launch on the
+    # stream it runs on -> per-kernel-class device times for phases_ms and the roofline objects
+    ea.profile_reset()
+    ea.profile_enable(True)
+    p0, p1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    p0.record(stream)
+    for _ in range(args.steps):
+        step()
+    p1.record(stream)
+    torch.cuda.synchronize()
+    prof = ea.profile_read()
+    ea.profile_enable(False)
+    profiled_ms = p0.elapsed_time(p1) / args.steps
 
     # roofline of the dominant kernel: FW phase-3 min-plus tiles (ALU bound)
     peaks = measured_peaks()
@@ -418,8 +459,34 @@ def run_ours(args, rank, world, local_rank):
         cpu = {"value": v, "unit": UNIT, "cores": thr, "kind": "oracle",
                "sample": f"Dijkstra from the first {nrows} sources of the uncontracted {args.config} graph "
                          f"({dt:.1f} s on {thr} threads); entries = sources x N"}
+        cpu.update(host_info())
+        cpu["cfg1_one_core"] = cfg1_one_core()
 
-    launches = int(prof["launches"])
+    seeds = None
+    if world == 1 and not args.no_seeds:   # seeds 0/1/2, median of 5 single-step times each
+        seeds = {"note": "median of 5 single-step device times after 1 warm-up step; seed 0 from the timed region",
+                 "0": {"median_ms": statistics.median(step_ms), "entries_per_s": g.n * g.n / (statistics.median(step_ms) / 1e3)}}
+        for sd in (1, 2):
+            gs = gg.config(args.config, sd)
+            ss, sd_, sw = (torch.as_tensor(x).to(dev) for x in (gs.src, gs.dst, gs.w))
+            o2 = torch.empty((gs.n, gs.n), dtype=torch.int32, device=dev)
+            run = lambda: ea.apsp_full(gs.n, ss, sd_, sw, out=o2, flags=flags, stream=stream)  # noqa: E731
+            run()
+            torch.cuda.synchronize()
+            ts = []
+            for _ in range(5):
+                a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                a.record(stream)
+                run()
+                b.record(stream)
+                torch.cuda.synchronize()
+                ts.append(a.elapsed_time(b))
+            med = statistics.median(ts)
+            seeds[str(sd)] = {"median_ms": med, "entries_per_s": gs.n * gs.n / (med / 1e3), "n_reduced":
+                              ea.ear_decompose(gs.n, ss, sd_, sw).info().n_reduced}
+            del o2
+            torch.cuda.empty_cache()
+
     if rank == 0:
         line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": K, "warmup": args.warmup,
                 "ms_per_step": ms_max / K, "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
@@ -437,7 +504,10 @@ def run_ours(args, rank, world, local_rank):
                 "roofline": roofline, "roofline_expand": roofline_expand,
                 "fw_minplus_gops": fw_minplus / (fw_ms / 1e3) / 1e9 if fw_ms > 0 else None,
                 "phases_ms": phases, "phase2_alternatives": alt, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks,
-                "gpu_launches": launches,
+                "gpu_launches": launches, "step_ms": step_ms, "seeds": seeds,
+                "profiled_pass": {"ms_per_step": profiled_ms, "note": "roofline objects and phases_ms come from this "
+                                  "separate pass of the same K steps with CUDA events around every library launch; "
+                                  "the headline value is timed with them off"},
                 "gpu_launches_note": "own kernels in the timed region (CUB sort/scan launches of Phase I excluded)",
                 "mteps_context": g.m * g.n / (ms_max / K / 1e3) / 1e6}
         print(json.dumps(line), flush=True)
@@ -466,6 +536,7 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-alt", action="store_true", help="skip the one-off SSSP Phase II timing")
     ap.add_argument("--cpu-seconds", type=float, default=15.0)
+    ap.add_argument("--no-seeds", action="store_true", help="skip the seed 1/2 medians (SURVEY 8.d)")
     args = ap.parse_args()
 
     rank = int(os.environ.get("RANK", "0"))

@@ -245,6 +245,41 @@ ear_status_t apsp_full_host_async(int32_t n, int64_t m, const int32_t *h_src, co
                                   int32_t *h_out, int64_t ldo, ear_comm_t comm, void *stream, ear_job_t *job);
 ear_status_t ear_job_wait(ear_job_t job);
 
+/* ---------------------------------------------------------------- Minimum cycle basis (paper sec. 3)
+ * MCB of G (a basis of the cycle space over GF(2) of minimum total weight; dimension
+ * f = m - n + k) -- of the canonical simple graph of the input (self-loops dropped, parallel edges ->
+ * lightest, reading C3) -- computed on the reduced graph G^r (Lemma 3.1: same weight and
+ * dimension; closed ears are self-loops and parallel chains parallel edges of G^r) by de Pina's
+ * Algorithm 2 with the paper's processing phase (sec. 3.3.2): shortest-path
+ * trees from every vertex of G^r (read off Phase II's APSP matrix), the Mehlhorn-Michail candidate
+ * cycles sorted by weight, per phase the labels of Algorithm 3, the first non-orthogonal
+ * candidate, and the witness update (the independence test).  The MCB weight is unique; which basis
+ * is returned is implementation-defined.  Inputs as ear_decompose (caller-owned DEVICE edge arrays);
+ * synchronises `stream` several times.  On success *out is a library-owned result (ear_mcb_destroy).
+ * Memory: about 28 * N_r^2 bytes plus 16 bytes per candidate cycle.  Errors: EAR_EINVAL,
+ * EAR_EOVERFLOW, EAR_ENOMEM, EAR_ECUDA. */
+typedef struct ear_mcb_s *ear_mcb_t;
+typedef struct {
+  int32_t dim;            /* f = m - n + k basis cycles (counted on G^r; equal for G, Lemma 3.1) */
+  int64_t weight;         /* W(MCB): the sum of the basis cycles' weights */
+  int32_t n_reduced;      /* vertices of G^r */
+  int64_t m_reduced;      /* edges of G^r: one per maximal degree-two chain + the direct edges */
+  int32_t components;     /* k */
+  int64_t n_candidates;   /* Mehlhorn-Michail candidate cycles */
+  int32_t tree_depth;     /* most edges on a shortest-path-tree path (label levels per phase) */
+} ear_mcb_info_t;
+ear_status_t ear_mcb(int32_t n, int64_t m, const int32_t *d_src, const int32_t *d_dst, const int32_t *d_w,
+                     void *stream, ear_mcb_t *out);
+ear_status_t ear_mcb_info(ear_mcb_t mcb, ear_mcb_info_t *info);
+/* The basis cycles' weights, in phase order, into a caller DEVICE array of info.dim int64. */
+ear_status_t ear_mcb_cycle_weights(ear_mcb_t mcb, int64_t *d_weights, void *stream);
+/* Post-processing (sec. 3.3.3): basis cycle i as a closed walk of G -- its vertices in caller
+ * ids, in order, the first not repeated at the end; every chain edge of G^r replaced by the chain.
+ * Writes min(len, cap) ids to d_verts (DEVICE) and the cycle's length to *len (host); cap = 0 queries
+ * the length.  Synchronises `stream`.  Errors: EAR_EINVAL (i out of [0, dim)). */
+ear_status_t ear_mcb_cycle(ear_mcb_t mcb, int32_t i, int32_t *d_verts, int32_t cap, int32_t *len, void *stream);
+void ear_mcb_destroy(ear_mcb_t mcb);
+
 /* ---------------------------------------------------------------- multi-GPU plumbing
  * Contiguous near-equal split of `rows` rows over nranks: rank gets [*begin, *end). */
 void ear_row_block(int32_t rows, int32_t nranks, int32_t rank, int32_t *begin, int32_t *end);

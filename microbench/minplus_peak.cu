@@ -1,7 +1,9 @@
 // Int32 min-plus issue-rate microbenchmark for sm_100a (roofline denominator for the FW kernels).
 // Each variant runs independent register-only chains of the form c_i = min(c_i, c_{i+1} + b)
 // (not idempotent, so the compiler cannot fold repeats).  Reported: min-plus ops/s over the whole
-// GPU and ops/clk/SM from clock64, so the figure can be rescaled to the SM clock seen in a run.
+// GPU, and ops/clk/SM over each SM's busy window -- from the first block start to the last block end
+// on that SM, both read from the SM's own clock64 (round 1 divided by the mean per-BLOCK window, which
+// undercounts cycles whenever blocks of an SM do not overlap exactly and gave inconsistent figures).
 #include <cstdio>
 #include <cstdint>
 #include <cuda_runtime.h>
@@ -59,7 +61,13 @@ __global__ void __launch_bounds__(256) mp_kernel(int* out, const int* in, int it
   #pragma unroll
   for (int i = 0; i < NACC; ++i) s ^= c[i];
   out[blockIdx.x * blockDim.x + threadIdx.x] = s;
-  if (threadIdx.x == 0) cyc[blockIdx.x] = t1 - t0;
+  if (threadIdx.x == 0) {
+    unsigned smid;
+    asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+    cyc[3 * blockIdx.x] = smid;
+    cyc[3 * blockIdx.x + 1] = t0;
+    cyc[3 * blockIdx.x + 2] = t1;
+  }
 }
 
 template <int V>
@@ -76,16 +84,34 @@ int run(const char* name, double ops_per_update, int nsm, int* d_out, int* d_in,
     CK(cudaEventSynchronize(e1));
     float ms; cudaEventElapsedTime(&ms, e0, e1); if (ms < best) best = ms;
   }
-  static long long h_cyc[148 * 64];
-  CK(cudaMemcpy(h_cyc, d_cyc, sizeof(long long) * blocks, cudaMemcpyDeviceToHost));
-  double mc = 0; for (int i = 0; i < blocks; ++i) mc += h_cyc[i]; mc /= blocks;
+  static long long h_cyc[3 * 148 * 64];
+  CK(cudaMemcpy(h_cyc, d_cyc, sizeof(long long) * 3 * blocks, cudaMemcpyDeviceToHost));
+  // per SM: busy window = last end - first start on that SM's clock; ops of the blocks that ran there
+  static long long lo[1024], hi[1024], nb[1024];
+  for (int i = 0; i < 1024; ++i) { lo[i] = -1; hi[i] = 0; nb[i] = 0; }
+  for (int b = 0; b < blocks; ++b) {
+    const int sm = (int)h_cyc[3 * b];
+    if (sm < 0 || sm >= 1024) continue;
+    if (lo[sm] < 0 || h_cyc[3 * b + 1] < lo[sm]) lo[sm] = h_cyc[3 * b + 1];
+    if (h_cyc[3 * b + 2] > hi[sm]) hi[sm] = h_cyc[3 * b + 2];
+    nb[sm]++;
+  }
   double updates = (double)blocks * threads * iters * NACC;
   double ops = updates * ops_per_update;
-  // blocks/SM = 8 resident (256 thr, few regs) -> per-SM ops per cycle of one block's window
-  double ops_per_clk_sm = (ops / nsm) / mc;
-  double eff_mhz = mc / (best * 1e-3) / 1e6;
-  printf("{\"variant\": \"%s\", \"ms\": %.3f, \"Tops_per_s\": %.3f, \"ops_per_clk_per_sm\": %.1f, \"eff_sm_mhz\": %.0f}\n",
-         name, best, ops / (best * 1e-3) / 1e12, ops_per_clk_sm, eff_mhz);
+  double ratio = 0, win = 0;
+  int used = 0;
+  for (int sm = 0; sm < 1024; ++sm)
+    if (nb[sm]) {
+      const double w = (double)(hi[sm] - lo[sm]);
+      ratio += (double)nb[sm] * threads * iters * NACC * ops_per_update / w;
+      win += w;
+      ++used;
+    }
+  double ops_per_clk_sm = ratio / used;           // mean over SMs of that SM's ops / its busy cycles
+  double eff_mhz = (win / used) / (best * 1e-3) / 1e6;   // busy cycles per SM / kernel time
+  printf("{\"variant\": \"%s\", \"ms\": %.3f, \"Tops_per_s\": %.3f, \"ops_per_clk_per_sm\": %.1f, \"eff_sm_mhz\": %.0f, "
+         "\"sms_used\": %d, \"blocks\": %d}\n",
+         name, best, ops / (best * 1e-3) / 1e12, ops_per_clk_sm, eff_mhz, used, blocks);
   return 0;
 }
 
@@ -103,7 +129,7 @@ int main() {
   printf("{\"gpu\": \"%s\", \"sms\": %d, \"cc\": \"%d.%d\"}\n", p.name, nsm, p.major, p.minor);
   int *d_out, *d_in; long long* d_cyc;
   CK(cudaMalloc(&d_out, sizeof(int) * nsm * 8 * 256));
-  CK(cudaMalloc(&d_cyc, sizeof(long long) * nsm * 8));
+  CK(cudaMalloc(&d_cyc, sizeof(long long) * 3 * nsm * 8));
   int h_in[128]; h_in[0] = 1; for (int i = 1; i < 128; ++i) h_in[i] = (i * 37) % 101 + 1;
   CK(cudaMalloc(&d_in, sizeof(h_in))); CK(cudaMemcpy(d_in, h_in, sizeof(h_in), cudaMemcpyHostToDevice));
   run<0>("viaddmnmx", 1.0, nsm, d_out, d_in, d_cyc);

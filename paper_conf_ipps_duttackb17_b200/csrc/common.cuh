@@ -74,6 +74,7 @@ struct ear_plan_s {
   int32_t n_chain_vertices = 0;
   // reduced arcs (both directions, before the P:90 min)
   int32_t *re_u = nullptr, *re_v = nullptr, *re_w = nullptr;
+  int32_t *re_x = nullptr;      // first vertex after re_u on the arc: the chain's first interior vertex, -1 if direct
   // reduced-graph CSR for the per-source SSSP Phase II (built on first use)
   int32_t *r_rowptr = nullptr, *r_col = nullptr, *r_w = nullptr;
   void *r_arcs = nullptr;       // packed (col, w) int2 arcs: ELL rows of r_ell_k per vertex, or CSR order

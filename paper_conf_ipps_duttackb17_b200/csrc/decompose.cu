@@ -235,10 +235,11 @@ __global__ void k_seg_fill(int32_t nc, const int32_t *head, const int32_t *segsc
 
 __global__ void k_seg_last(int32_t nseg, int32_t nc, int32_t *seg_start) { seg_start[nseg] = nc; }
 
-// reduced arcs: tail terminal u, end terminal e != u (closed ears dropped, C6)
-__global__ void k_reduced_arcs(int64_t A, const int32_t *asrc, const int32_t *term, const int32_t *scan,
-                               RankBuf b, int32_t *ru, int32_t *rv, int32_t *rw, unsigned long long *count,
-                               int emit) {
+// reduced arcs: tail terminal u, end terminal e != u (closed ears dropped, C6); rx: the first vertex
+// after u (the chain's first interior vertex), or -1 when the arc is a direct terminal-terminal edge
+__global__ void k_reduced_arcs(int64_t A, const int32_t *asrc, const int32_t *adst, const int32_t *term,
+                               const int32_t *scan, RankBuf b, int32_t *ru, int32_t *rv, int32_t *rw, int32_t *rx,
+                               unsigned long long *count, int emit) {
   GRID_STRIDE(a, A) {
     int32_t u = asrc[a];
     if (term[u]) {
@@ -249,6 +250,7 @@ __global__ void k_reduced_arcs(int64_t A, const int32_t *asrc, const int32_t *te
           ru[k] = scan[u];
           rv[k] = scan[e];
           rw[k] = (int32_t)b.sum[a];
+          rx[k] = term[adst[a]] ? -1 : adst[a];
         }
       }
     }
@@ -299,7 +301,7 @@ struct Scratch {
 // and are released in stream order on the stream the plan was created on.
 void plan_free(ear_plan_s *p) {
   if (!p) return;
-  void *arrs[] = {p->desc, p->tid, p->ear, p->seg_of, p->seg_start, p->seg_vert, p->re_u, p->re_v, p->re_w,
+  void *arrs[] = {p->desc, p->tid, p->ear, p->seg_of, p->seg_start, p->seg_vert, p->re_u, p->re_v, p->re_w, p->re_x,
                   p->r_rowptr, p->r_col, p->r_w, p->r_arcs};
   for (void *a : arrs)
     if (a) cudaFreeAsync(a, p->stream);
@@ -489,7 +491,9 @@ ear_status_t decompose(int32_t n, int64_t m, const int32_t *src, const int32_t *
   unsigned long long *d_rcount;
   EAR_TRY(S.alloc(&d_rcount, 1));
   EAR_CUDA_TRY(dev_memset(d_rcount, 0, sizeof(unsigned long long), st));
-  if (A > 0) EAR_LAUNCH(k_reduced_arcs, grid_for(A), NT, 0, st)(A, asrc, term, scan, rb[cur], nullptr, nullptr, nullptr, d_rcount, 0);
+  if (A > 0)
+    EAR_LAUNCH(k_reduced_arcs, grid_for(A), NT, 0, st)(A, asrc, adst, term, scan, rb[cur], nullptr, nullptr, nullptr,
+                                                       nullptr, d_rcount, 0);
   unsigned long long h_rcount = 0;
   int32_t h_stats[2];
   EAR_CUDA_TRY(rbk.get(&h_rcount, d_rcount, sizeof(h_rcount)));
@@ -502,10 +506,11 @@ ear_status_t decompose(int32_t n, int64_t m, const int32_t *src, const int32_t *
   EAR_TRY(plan_alloc(&plan->re_u, plan->n_redges, st));
   EAR_TRY(plan_alloc(&plan->re_v, plan->n_redges, st));
   EAR_TRY(plan_alloc(&plan->re_w, plan->n_redges, st));
+  EAR_TRY(plan_alloc(&plan->re_x, plan->n_redges, st));
   EAR_CUDA_TRY(dev_memset(d_rcount, 0, sizeof(unsigned long long), st));
   if (A > 0)
-    EAR_LAUNCH(k_reduced_arcs, grid_for(A), NT, 0, st)(A, asrc, term, scan, rb[cur], plan->re_u, plan->re_v, plan->re_w,
-                                              d_rcount, 1);
+    EAR_LAUNCH(k_reduced_arcs, grid_for(A), NT, 0, st)(A, asrc, adst, term, scan, rb[cur], plan->re_u, plan->re_v,
+                                                       plan->re_w, plan->re_x, d_rcount, 1);
 
   // same-chain vertex lists sorted by (chain id, off_left)
   const int32_t nc = n - plan->n_reduced;
