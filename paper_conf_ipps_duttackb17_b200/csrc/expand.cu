@@ -30,6 +30,8 @@
 // gathers go to HBM at the first touch of each sector and their latency is what bounds the kernel;
 // with D resident in L2 the same kernel runs at ~90 % of the copy bandwidth.
 // k_same_chain: the P:107 along-chain patch, one warp per row, touching only same-chain entries.
+#include <cub/cub.cuh>
+
 #include <algorithm>
 #include <cstdlib>
 
@@ -257,21 +259,51 @@ __global__ void k_same_chain(const VDesc *__restrict__ desc, const int32_t *__re
 
 // Compact / query mode: S[s,t] for arbitrary pairs from D and the descriptors
 // alone -- UPDATE_DISTANCE evaluated per pair, O(N_r^2 + N) memory instead of N^2.
+__device__ __forceinline__ int32_t query_one(const int32_t *__restrict__ D, int64_t ldd, const VDesc *__restrict__ desc,
+                                             const int32_t *__restrict__ ear, int32_t s, int32_t t) {
+  const VDesc a = desc[s], b = desc[t];
+  const int32_t *Dp = D + (int64_t)a.p * ldd, *Dq = D + (int64_t)a.q * ldd;
+  // R[e,t] for e in {p_s, q_s} (2-term), then the 4-term rule
+  const int32_t rp = min(__viaddmin_s32(Dp[b.q], b.cq, Dp[b.p] + b.cp), INF);
+  const int32_t rq = min(__viaddmin_s32(Dq[b.q], b.cq, Dq[b.p] + b.cp), INF);
+  int32_t v = min(__viaddmin_s32(a.cq, rq, a.cp + rp), INF);
+  const int32_t es = ear[s];
+  if (es >= 0 && es == ear[t]) v = min(v, abs(a.cp - b.cp));   // same chain (C8/C9)
+  return v;
+}
 __global__ void k_query_pairs(const int32_t *__restrict__ D, int64_t ldd, const VDesc *__restrict__ desc,
                               const int32_t *__restrict__ ear, int64_t npairs, const int32_t *__restrict__ qs,
                               const int32_t *__restrict__ qt, int32_t *__restrict__ out) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < npairs; i += (int64_t)gridDim.x * blockDim.x)
+    out[i] = query_one(D, ldd, desc, ear, qs[i], qt[i]);
+}
+
+// Bucketed query: the pairs are first grouped by the source's left chain end p_s (a counting sort over
+// the N_r terminals: histogram, scan, scatter of packed (s, t, i) records), so that the pairs of one
+// bucket -- read consecutively -- share the D row p_s (and mostly q_s) while it sits in L2; the random
+// D sectors of the per-pair kernel become L2 hits.  out[i] keeps the caller's pair order.
+__global__ void k_qhist(int64_t npairs, const int32_t *__restrict__ qs, const VDesc *__restrict__ desc, int32_t *hist) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < npairs; i += (int64_t)gridDim.x * blockDim.x)
+    atomicAdd(&hist[desc[qs[i]].p], 1);
+}
+__global__ void k_qscatter(int64_t npairs, const int32_t *__restrict__ qs, const int32_t *__restrict__ qt,
+                           const VDesc *__restrict__ desc, int64_t *cur, int4 *rec) {
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < npairs; i += (int64_t)gridDim.x * blockDim.x) {
-    const int32_t s = qs[i], t = qt[i];
-    const VDesc a = desc[s], b = desc[t];
-    const int32_t *Dp = D + (int64_t)a.p * ldd, *Dq = D + (int64_t)a.q * ldd;
-    // R[e,t] for e in {p_s, q_s} (2-term), then the 4-term rule
-    const int32_t rp = min(__viaddmin_s32(Dp[b.q], b.cq, Dp[b.p] + b.cp), INF);
-    const int32_t rq = min(__viaddmin_s32(Dq[b.q], b.cq, Dq[b.p] + b.cp), INF);
-    int32_t v = min(__viaddmin_s32(a.cq, rq, a.cp + rp), INF);
-    const int32_t es = ear[s];
-    if (es >= 0 && es == ear[t]) v = min(v, abs(a.cp - b.cp));   // same chain (C8/C9)
-    out[i] = v;
+    const int32_t s = qs[i];
+    const int64_t pos = atomicAdd(reinterpret_cast<unsigned long long *>(&cur[desc[s].p]), 1ull);
+    rec[pos] = make_int4(s, qt[i], (int32_t)(i & 0xFFFFFFFF), (int32_t)(i >> 32));
   }
+}
+__global__ void k_query_bucketed(const int32_t *__restrict__ D, int64_t ldd, const VDesc *__restrict__ desc,
+                                 const int32_t *__restrict__ ear, int64_t npairs, const int4 *__restrict__ rec,
+                                 int32_t *__restrict__ out) {
+  for (int64_t j = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; j < npairs; j += (int64_t)gridDim.x * blockDim.x) {
+    const int4 r = rec[j];
+    out[(int64_t)(uint32_t)r.z | ((int64_t)r.w << 32)] = query_one(D, ldd, desc, ear, r.x, r.y);
+  }
+}
+__global__ void k_hist64(int32_t nb, const int32_t *hist, int64_t *h64) {
+  for (int32_t b = blockIdx.x * blockDim.x + threadIdx.x; b < nb; b += gridDim.x * blockDim.x) h64[b] = hist[b];
 }
 
 
@@ -311,11 +343,48 @@ ear_status_t expand(const ear_plan_s *plan, const int32_t *D, int64_t ldd, int32
   return EAR_OK;
 }
 
+// Bucketing pays once a batch has many pairs per terminal row (EAR_QUERY_BUCKET_MIN overrides the
+// threshold; 0 disables bucketing).
 ear_status_t query_pairs(const ear_plan_s *plan, const int32_t *D, int64_t ldd, int64_t npairs, const int32_t *qs,
                          const int32_t *qt, int32_t *out, cudaStream_t st) {
   if (npairs <= 0) return EAR_OK;
   const int grid = (int)std::min<int64_t>(ceil_div(npairs, 256), 148 * 16);
-  EAR_LAUNCH(k_query_pairs, grid, 256, 0, st)(D, ldd, plan->desc, plan->ear, npairs, qs, qt, out);
+  const char *env = getenv("EAR_QUERY_BUCKET_MIN");
+  const int64_t min_pairs = env ? atoll(env) : (int64_t)4 * plan->n_reduced + (1 << 20);
+  if (min_pairs <= 0 || npairs < min_pairs) {
+    EAR_LAUNCH(k_query_pairs, grid, 256, 0, st)(D, ldd, plan->desc, plan->ear, npairs, qs, qt, out);
+    EAR_CUDA_TRY(cudaGetLastError());
+    return EAR_OK;
+  }
+  const int32_t nb = std::max(plan->n_reduced, 1);
+  int32_t *hist = nullptr;
+  int64_t *h64 = nullptr, *start = nullptr;
+  int4 *rec = nullptr;
+  void *tmp = nullptr;
+  size_t tb = 0;
+  EAR_CUDA_TRY(cub::DeviceScan::ExclusiveSum(nullptr, tb, h64, start, nb, st));
+  ear_status_t s = EAR_OK;
+  if (cudaMallocAsync((void **)&hist, sizeof(int32_t) * nb, st) != cudaSuccess ||
+      cudaMallocAsync((void **)&h64, sizeof(int64_t) * nb, st) != cudaSuccess ||
+      cudaMallocAsync((void **)&start, sizeof(int64_t) * nb, st) != cudaSuccess ||
+      cudaMallocAsync(&tmp, std::max<size_t>(tb, 16), st) != cudaSuccess ||
+      cudaMallocAsync((void **)&rec, sizeof(int4) * (size_t)npairs, st) != cudaSuccess) {
+    cudaGetLastError();
+    s = EAR_ENOMEM;
+    set_error("ear_query_pairs: out of device memory for the buckets");
+  }
+  if (s == EAR_OK) {
+    const int gb = (int)std::min<int64_t>(ceil_div(nb, 256), 148 * 16);
+    EAR_CUDA_TRY(dev_memset(hist, 0, sizeof(int32_t) * nb, st));
+    EAR_LAUNCH(k_qhist, grid, 256, 0, st)(npairs, qs, plan->desc, hist);
+    EAR_LAUNCH(k_hist64, gb, 256, 0, st)(nb, hist, h64);
+    EAR_CUDA_TRY(cub::DeviceScan::ExclusiveSum(tmp, tb, h64, start, nb, st));
+    EAR_LAUNCH(k_qscatter, grid, 256, 0, st)(npairs, qs, qt, plan->desc, start, rec);
+    EAR_LAUNCH(k_query_bucketed, grid, 256, 0, st)(D, ldd, plan->desc, plan->ear, npairs, rec, out);
+  }
+  for (void *p : {(void *)hist, (void *)h64, (void *)start, tmp, (void *)rec})
+    if (p) cudaFreeAsync(p, st);
+  EAR_TRY(s);
   EAR_CUDA_TRY(cudaGetLastError());
   return EAR_OK;
 }

@@ -67,6 +67,12 @@ class _BccInfo(ctypes.Structure):
                 ("rereduce_levels", ctypes.c_int32)]
 
 
+class _McbInfo(ctypes.Structure):
+    _fields_ = [("dim", ctypes.c_int32), ("weight", ctypes.c_int64), ("n_reduced", ctypes.c_int32),
+                ("m_reduced", ctypes.c_int64), ("components", ctypes.c_int32), ("n_candidates", ctypes.c_int64),
+                ("tree_depth", ctypes.c_int32)]
+
+
 # (name, restype, argtypes) for every symbol declared in include/ear_apsp.h
 _P, _I32, _I64, _U32 = ctypes.c_void_p, ctypes.c_int32, ctypes.c_int64, ctypes.c_uint32
 SIGNATURES = {
@@ -87,6 +93,11 @@ SIGNATURES = {
     "apsp_full_host": (_I32, [_I32, _I64, _P, _P, _P, _U32, _I32, _I32, _P, _I64, _P, _P]),
     "apsp_full_host_async": (_I32, [_I32, _I64, _P, _P, _P, _U32, _I32, _I32, _P, _I64, _P, _P, ctypes.POINTER(_P)]),
     "ear_job_wait": (_I32, [_P]),
+    "ear_mcb": (_I32, [_I32, _I64, _P, _P, _P, _P, ctypes.POINTER(_P)]),
+    "ear_mcb_info": (_I32, [_P, ctypes.POINTER(_McbInfo)]),
+    "ear_mcb_cycle_weights": (_I32, [_P, _P, _P]),
+    "ear_mcb_cycle": (_I32, [_P, _I32, _P, _I32, ctypes.POINTER(_I32), _P]),
+    "ear_mcb_destroy": (None, [_P]),
     "ear_row_block": (None, [_I32, _I32, _I32, ctypes.POINTER(_I32), ctypes.POINTER(_I32)]),
     "ear_comm_init": (_I32, [_I32, _I32, _P, _P, ctypes.POINTER(_P)]),
     "ear_comm_info": (_I32, [_P, ctypes.POINTER(_I32), ctypes.POINTER(_I32)]),
@@ -417,6 +428,54 @@ def apsp_full_host_async(n: int, src, dst, w, out: torch.Tensor | None = None, r
                                       flags, row_begin, row_end, out.data_ptr(), out.stride(0), _comm_handle(comm),
                                       _stream(stream), ctypes.byref(h)), "apsp_full_host_async")
     return HostJob(h, out, tens)
+
+
+class Mcb:
+    """Minimum cycle basis of G (paper sec. 3) computed on G^r (library-owned result)."""
+
+    def __init__(self, handle, n):
+        self.handle, self.n = handle, n
+
+    def info(self) -> dict:
+        i = _McbInfo()
+        _check(lib().ear_mcb_info(self.handle, ctypes.byref(i)), "ear_mcb_info")
+        return {f: getattr(i, f) for f, _ in _McbInfo._fields_}
+
+    def weights(self, stream=None) -> torch.Tensor:
+        """The basis cycles' weights in phase order (int64, on the device)."""
+        f = self.info()["dim"]
+        out = torch.empty(max(f, 1), dtype=torch.int64, device="cuda")
+        _check(lib().ear_mcb_cycle_weights(self.handle, out.data_ptr(), _stream(stream)), "ear_mcb_cycle_weights")
+        return out[:f]
+
+    def cycle(self, i: int, stream=None) -> torch.Tensor:
+        """Post-processing (sec. 3.3.3): basis cycle i as a closed walk of G, caller vertex ids."""
+        n = _I32()
+        _check(lib().ear_mcb_cycle(self.handle, i, None, 0, ctypes.byref(n), _stream(stream)), "ear_mcb_cycle")
+        out = torch.empty(max(n.value, 1), dtype=torch.int32, device="cuda")
+        _check(lib().ear_mcb_cycle(self.handle, i, out.data_ptr(), n.value, ctypes.byref(n), _stream(stream)),
+               "ear_mcb_cycle")
+        return out[:n.value]
+
+    def destroy(self):
+        if self.handle:
+            lib().ear_mcb_destroy(self.handle)
+            self.handle = None
+
+    def __del__(self):  # pragma: no cover
+        try:
+            self.destroy()
+        except Exception:
+            pass
+
+
+def mcb(n: int, src: torch.Tensor, dst: torch.Tensor, w: torch.Tensor, stream=None) -> Mcb:
+    """Minimum cycle basis of the graph (device edge arrays), by the paper's sec. 3 method on G^r."""
+    src, dst, w = _dev_i32(src, "src"), _dev_i32(dst, "dst"), _dev_i32(w, "w")
+    h = _P()
+    _check(lib().ear_mcb(n, src.numel(), src.data_ptr(), dst.data_ptr(), w.data_ptr(), _stream(stream),
+                         ctypes.byref(h)), "ear_mcb")
+    return Mcb(h, n)
 
 
 def profile_enable(on: bool = True):

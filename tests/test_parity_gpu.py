@@ -362,6 +362,27 @@ def test_query_pairs_cfg4_without_full_matrix(pkg):
     assert_exact(got, ref[:, cols], "cfg4 query pairs")
 
 
+@pytest.mark.parametrize("bucket", ["forced", "off"])
+@pytest.mark.parametrize("name", ["corner", "cfg2"])
+def test_query_pairs_bucketed(pkg, monkeypatch, name, bucket):
+    """The bucketed query path (pairs grouped by the source's chain end; EAR_QUERY_BUCKET_MIN=1 forces it
+    for any batch) and the per-pair path (0), shuffled pair order, against oracle rows."""
+    monkeypatch.setenv("EAR_QUERY_BUCKET_MIN", "1" if bucket == "forced" else "0")
+    g = gg.corner_cases(44, n_target=700) if name == "corner" else gg.config("cfg2")
+    plan = pkg.ear_decompose(g.n, dev(g.src), dev(g.dst), dev(g.w), flags=pkg.FLAG_BCC)
+    D = pkg.alloc_D(plan)
+    pkg.apsp_reduced(plan, D)
+    rng = np.random.default_rng(17)
+    rows = rng.choice(g.n, min(g.n, 30), replace=False)
+    ref = oracle.apsp_rows(g.n, g.src, g.dst, g.w, rows)
+    s = np.repeat(rows, g.n).astype(np.int32)
+    t = np.tile(np.arange(g.n), len(rows)).astype(np.int32)
+    perm = rng.permutation(len(s))
+    got = np.empty(len(s), np.int32)
+    got[perm] = pkg.query_pairs(plan, D, dev(s[perm]), dev(t[perm])).cpu().numpy()
+    assert_exact(got.reshape(len(rows), g.n), ref, f"bucketed query {name} {bucket}")
+
+
 # ------------------------------------------------------------------------------ NEXT 2: SSSP Phase II
 @pytest.mark.parametrize("seed", range(12))
 def test_sssp_phase2_corner_cases(pkg, seed):

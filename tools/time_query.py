@@ -1,13 +1,10 @@
-#!/usr/bin/env python
-"""Compact / query mode (UPDATE_DISTANCE per pair; memory P:137) measured:
-Phases I-II once (D of G^r kept, O(N_r^2 + N) memory instead of N^2), then ear_query_pairs on batches
-of uniformly random (s, t) pairs.  Each pair reads two 16-byte descriptors, two chain ids and four D
-entries at random addresses, plus 12 streamed bytes (s, t, result).  The descriptors and chain ids
-(20 bytes per vertex: 2 MB at cfg4, 4 MB at cfg5) stay in L2; D (3.6 / 14.4 GB) does not, so the DRAM
-traffic is 4 random 32-byte D sectors + 12 bytes per pair, reported as dram_GBps against the copy
-bandwidth (random sectors cannot reach the streaming rate).  Parity of the query path: tests/test_parity_gpu.py.
+"""Query mode throughput (S[s,t] for arbitrary pairs from D + descriptors, no N x N
+matrix): 2^26 pairs per batch on cfg4 (or the given config), uniformly random and source-grouped
+(1,024 random targets per random source), through ear_query_pairs with its bucketing by the source's
+chain end (default) and with bucketing disabled (EAR_QUERY_BUCKET_MIN=0).  Parity of the query path:
+tests/test_parity_gpu.py.
 
-    python tools/time_query.py [cfg4|cfg5] [--pairs 67108864] [--reps 5]
+    python tools/time_query.py [cfg4] [--pairs N] [--out profiles/...jsonl]
 """
 import argparse
 import json
@@ -28,8 +25,8 @@ def main():
     ap.add_argument("config", nargs="?", default="cfg4")
     ap.add_argument("--pairs", type=int, default=1 << 26)
     ap.add_argument("--reps", type=int, default=5)
+    ap.add_argument("--out", default=None)
     args = ap.parse_args()
-
     g = gg.config(args.config)
     src, dst, w = (torch.as_tensor(x).cuda() for x in (g.src, g.dst, g.w))
     plan = ea.ear_decompose(g.n, src, dst, w, flags=ea.FLAG_BCC)
@@ -37,24 +34,44 @@ def main():
     ea.apsp_reduced(plan, D)
     torch.cuda.synchronize()
     gen = torch.Generator(device="cuda").manual_seed(7)
-    s = torch.randint(0, g.n, (args.pairs,), device="cuda", dtype=torch.int32, generator=gen)
-    t = torch.randint(0, g.n, (args.pairs,), device="cuda", dtype=torch.int32, generator=gen)
-    out = torch.empty(args.pairs, dtype=torch.int32, device="cuda")
-    ea.query_pairs(plan, D, s, t, out=out)   # warm-up
-    torch.cuda.synchronize()
-    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    e0.record()
-    for _ in range(args.reps):
-        ea.query_pairs(plan, D, s, t, out=out)
-    e1.record()
-    torch.cuda.synchronize()
-    ms = e0.elapsed_time(e1) / args.reps
+    P = args.pairs
+    workloads = {
+        "uniform": (torch.randint(0, g.n, (P,), device="cuda", dtype=torch.int32, generator=gen),
+                    torch.randint(0, g.n, (P,), device="cuda", dtype=torch.int32, generator=gen)),
+        "source_grouped_1024": (torch.randint(0, g.n, (P // 1024,), device="cuda", dtype=torch.int32,
+                                              generator=gen).repeat_interleave(1024),
+                                torch.randint(0, g.n, (P,), device="cuda", dtype=torch.int32, generator=gen)),
+    }
+    out = torch.empty(P, dtype=torch.int32, device="cuda")
     peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
-    dram_bytes = (4 * 32 + 12) * args.pairs
-    print(json.dumps({"config": args.config, "n": g.n, "n_reduced": plan.info().n_reduced,
-                      "D_bytes": int(D.numel()) * 4, "full_matrix_bytes": 4 * g.n * g.n,
-                      "pairs": args.pairs, "ms_per_batch": ms, "pairs_per_s": args.pairs / (ms / 1e3),
-                      "dram_GBps": dram_bytes / (ms / 1e3) / 1e9, "hbm_copy_GBps": peaks["hbm_gbs"]}))
+    lines = []
+    for name, (s, t) in workloads.items():
+        res = {}
+        for mode in ("per_pair", "bucketed"):
+            os.environ["EAR_QUERY_BUCKET_MIN"] = "0" if mode == "per_pair" else "1"
+            ea.query_pairs(plan, D, s, t, out=out)
+            torch.cuda.synchronize()
+            ref = out.clone() if mode == "per_pair" else ref
+            same = bool(torch.equal(out, ref))
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record()
+            for _ in range(args.reps):
+                ea.query_pairs(plan, D, s, t, out=out)
+            e1.record()
+            torch.cuda.synchronize()
+            ms = e0.elapsed_time(e1) / args.reps
+            res[mode] = {"ms_per_batch": ms, "pairs_per_s": P / (ms / 1e3), "same_as_per_pair": same}
+        os.environ.pop("EAR_QUERY_BUCKET_MIN", None)
+        rec = {"config": args.config, "workload": name, "pairs": P, "n": g.n, "n_reduced": plan.info().n_reduced,
+               "D_bytes": int(D.numel()) * 4, "full_matrix_bytes": 4 * g.n * g.n, **res,
+               "speedup": res["per_pair"]["ms_per_batch"] / res["bucketed"]["ms_per_batch"],
+               "hbm_copy_GBps": peaks.get("hbm_gbs")}
+        print(json.dumps(rec), flush=True)
+        lines.append(rec)
+    if args.out:
+        with open(args.out, "w") as f:
+            for r in lines:
+                f.write(json.dumps(r) + "\n")
 
 
 if __name__ == "__main__":
