@@ -380,7 +380,7 @@ def run_ours(args, rank, world, local_rank):
               "expand": ex_ms / K, "same_chain": prof["same_chain_ms"] / K,
               "bcc_pieces": prof["bcc_pieces_ms"] / K, "compose": prof["compose_ms"] / K,
               "fw16_conv": prof["fw16_conv_ms"] / K, "rereduce": prof["rereduce_ms"] / K,
-              "bcc_prepare": prof["bcc_prepare_ms"] / K,
+              "bcc_prepare": prof["bcc_prepare_ms"] / K, "expand_d16": prof["expand_d16_ms"] / K,
               "fw_side_overlapped": prof["fw_side_ms"] / K}
     fw_minplus = prof["fw_phase2_minplus"] + prof["fw_phase3_minplus"]
     del out

@@ -23,7 +23,8 @@
  *   - Return value: EAR_OK or a negative ear_status_t; nothing throws.  ear_last_error() returns a
  *     thread-local human-readable message for the last failure.
  *   - Asynchronous on `stream` unless stated.  Kernel faults surface as EAR_ECUDA at the next
- *     synchronising call.  A plan is not thread-safe; distinct plans are.
+ *     synchronising call.  A plan is not thread-safe; distinct plans are (every FW call owns its
+ *     lookahead side stream, events and tile counters: tests/test_concurrency_gpu.py).
  */
 #ifndef EAR_APSP_H
 #define EAR_APSP_H
@@ -129,11 +130,14 @@ void ear_plan_destroy(ear_plan_t plan);
  *   comm != NULL (P ranks, even P = 1): d_D holds this rank's OWNED TILE ROWS -- the 128-row blocks
  *                 ti with (ti mod 2P) in {rank, 2P-1-rank} (a zig-zag that balances the upper
  *                 triangle), in ascending order, ear_owned_tile_rows() blocks of 128 rows x ldd.  Each
- *                 round the pivot row block is assembled on every rank by an NCCL all-reduce(MIN) of
- *                 the owners' pieces, closed locally, and every rank updates only its owned UPPER
- *                 tiles: the single-GPU symmetric halving of the work survives the sharding
- *                 (DESIGN.md "Multi-GPU").  Only the upper tiles of d_D are meaningful afterwards;
- *                 ear_gather_reduced assembles the full symmetric matrix.
+ *                 round the owner of row k closes the pivot tile and stores it into every peer's window,
+ *                 every rank applies phase 2 to the pieces of the pivot row block it holds and stores them
+ *                 into every rank's window (the per-round broadcast of the pieces: each rank receives the
+ *                 rest of the block once), and every rank updates only its owned UPPER tiles: the
+ *                 single-GPU symmetric halving of the work survives the sharding.  Only
+ *                 the upper tiles of d_D are meaningful afterwards; ear_gather_reduced assembles the full
+ *                 symmetric matrix.  Collective over the communicator's ranks (may call its all-gather
+ *                 callback when the exchange window must grow).
  * Asynchronous.  Errors: EAR_EINVAL (ldd too small/misaligned), EAR_ENCCL, EAR_ECUDA. */
 ear_status_t apsp_reduced(ear_plan_t plan, int32_t *d_D, int64_t ldd, ear_comm_t comm, void *stream);
 
@@ -147,11 +151,10 @@ ear_status_t apsp_reduced_emulated(ear_plan_t plan, int32_t nranks, int32_t *d_D
                                    void *stream);
 
 /* DIAGNOSTIC, produces no result: the device work of ONE rank `rank` of an `nranks`-rank run of the
- * packed 16-bit sharded FW (sec. 7 of DESIGN.md) on the current device -- narrowing its owned rows,
- * and per round the pivot-row widening, the int32 phases 1-2, the narrowing and the packed phase 3 on
- * its owned upper tiles -- without the other ranks and without the exchange (the pivot row block then
- * holds only this rank's pieces; min-plus work is data-independent, so the time is that rank's
- * compute).  Used to measure per-rank compute scaling on one GPU (tools/rank_timing.py).  Allocates
+ * sharded FW (sec. 7 of DESIGN.md) on the current device -- packed u16x2, or int32 when the plan was made
+ * with EAR_FLAG_FW32 -- per round its pivot pieces, phase 1 when it owns the pivot, phase 2 on its pieces
+ * and phase 3 on its owned upper tiles, without the other ranks and without the exchange (min-plus work
+ * is data-independent, so the time is that rank's compute).  Used to measure per-rank compute scaling on one GPU (tools/rank_timing.py).  Allocates
  * and frees its own scratch; asynchronous.  Errors: EAR_EINVAL (NULL plan, rank out of range),
  * EAR_ENOMEM, EAR_ECUDA. */
 ear_status_t apsp_reduced_rank_timing(ear_plan_t plan, int32_t nranks, int32_t rank, void *stream);
@@ -161,9 +164,10 @@ ear_status_t apsp_reduced_rank_timing(ear_plan_t plan, int32_t nranks, int32_t r
 int32_t ear_owned_tile_rows(int32_t n_reduced_padded, int32_t nranks, int32_t rank);
 
 /* Assemble the full Np x Np matrix d_D_full (ldd_full >= Np) from every rank's owned storage written
- * by apsp_reduced with `comm`: each rank scatters its upper tiles and their mirrors into an
- * INF-filled matrix, and one NCCL all-reduce(MIN) combines them.  d_D_block must not alias
- * d_D_full.  Without comm, a plain copy. */
+ * by apsp_reduced with `comm` (the all-gather of D): each rank's owned rows are placed in its exchange
+ * window, and every rank reads every tile from the window of the rank that owns it -- the lower
+ * triangle as the transpose of the upper tile, so no mirror pass follows -- between two stream-ordered
+ * barriers.  d_D_block must not alias d_D_full.  Without comm, a plain copy.  Collective. */
 ear_status_t ear_gather_reduced(ear_plan_t plan, const int32_t *d_D_block, int64_t ldd_block,
                                 int32_t *d_D_full, int64_t ldd_full, ear_comm_t comm, void *stream);
 
@@ -341,6 +345,8 @@ typedef struct {
   int64_t fw16_prechecked;     /* packed FWs abandoned after round 3: the eccentricity of reduced vertex 0
                                   (one SSSP row, overlapped with rounds 0-3) already reached the 16-bit cap;
                                   each is also counted in fw16_fallbacks */
+  double expand_d16_ms;        /* pair-major expansion: D narrowed to the u16 rows it stages (with the range
+                                  check), before the k_expand_pairs launch timed in expand_ms */
 } ear_profile_t;
 
 void ear_profile_enable(int32_t on);

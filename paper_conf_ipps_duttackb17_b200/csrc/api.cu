@@ -279,35 +279,84 @@ ear_status_t ear_query_pairs(ear_plan_t p, const int32_t *d_D_full, int64_t ldd,
   return query_pairs(p, d_D_full, ldd, npairs, d_s, d_t, d_out, (cudaStream_t)stream);
 }
 
+// D as Phase III reads it: the int32 Np x Np matrix, or -- on the single-GPU Phase II by blocks, when
+// the pair-major expansion applies and every distance fits -- only its u16 rows (half the bytes, and the
+// expansion stages them without a narrowing pass)
+struct DKeep {
+  int32_t *D = nullptr;
+  uint16_t *D16 = nullptr;
+  int32_t ld16 = 0;
+};
+
+static ear_status_t expand_kept(ear_plan_s *p, const DKeep &k, int32_t Np, int32_t r0, int32_t r1, int32_t *out,
+                                int64_t ldo, cudaStream_t st) {
+  if (k.D16) return expand_from16(p, k.D16, k.ld16, r0, r1, out, ldo, st);
+  return expand(p, k.D, Np, r0, r1, out, ldo, st);
+}
+
+static void free_kept(DKeep &k, cudaStream_t st) {
+  if (k.D) cudaFreeAsync(k.D, st);
+  if (k.D16) cudaFreeAsync(k.D16, st);
+  k = DKeep{};
+}
+
 // Phases II + III for an existing plan into device rows (shared by apsp_full / apsp_full_host).
+// `u16_ok`: the rows Phase III will write are 16-byte aligned with ldo % 4 == 0 (the pair-major kernel's
+// stores).  With `keep` D is handed back (not freed) for later expansions.
 static ear_status_t solve_rows(ear_plan_s *p, int32_t row_begin, int32_t row_end, int32_t *d_out, int64_t ldo,
-                               ear_comm_t comm, cudaStream_t st, int32_t **D_keep) {
+                               ear_comm_t comm, cudaStream_t st, DKeep *keep, bool u16_ok) {
   const int32_t P = comm ? comm->nranks : 1;
   const int32_t Np = padded(p, P);
-  int32_t *D = nullptr, *Dfull = nullptr;
+  DKeep k;
   ear_status_t s = EAR_OK;
-  if (!comm) {
-    EAR_CUDA_TRY(cudaMallocAsync((void **)&D, sizeof(int32_t) * (size_t)Np * Np, st));
-    s = apsp_reduced(p, D, Np, nullptr, st);
-    Dfull = D;
-  } else if (p->flags & EAR_FLAG_BCC) {
-    // every rank holds every solved piece after bcc_solve: compose the full matrix directly, no gather
-    EAR_CUDA_TRY(cudaMallocAsync((void **)&Dfull, sizeof(int32_t) * (size_t)Np * Np, st));
-    s = bcc_solve(p, comm, Dfull, Np, Np, 0, Np, nullptr, st);
-  } else {
-    // the owned rows live in this rank's exchange window, where the gather reads them
-    EAR_CUDA_TRY(cudaMallocAsync((void **)&Dfull, sizeof(int32_t) * (size_t)Np * Np, st));
-    s = fw_shard_buffer(comm, Np, st, &D);
-    if (s == EAR_OK) s = apsp_reduced(p, D, Np, comm, st);
-    if (s == EAR_OK) s = ear_gather_reduced(p, D, Np, Dfull, Np, comm, st);
+  if (!comm && (p->flags & EAR_FLAG_BCC) && u16_ok && xp_applicable(p, st)) {
+    k.ld16 = xp_row_stride(p);
+    int32_t *flag = nullptr;
+    EAR_CUDA_TRY(cudaMallocAsync((void **)&k.D16, sizeof(uint16_t) * (size_t)p->n_reduced * k.ld16, st));
+    EAR_CUDA_TRY(cudaMallocAsync((void **)&flag, sizeof(int32_t), st));
+    EAR_CUDA_TRY(dev_memset(flag, 0, sizeof(int32_t), st));
+    s = bcc_solve(p, nullptr, nullptr, Np, Np, 0, p->n_reduced, nullptr, st, k.D16, k.ld16, flag);
+    int32_t h_flag = 1;
+    if (s == EAR_OK) {
+      Readback rb(st);
+      cudaError_t e = rb.get(&h_flag, flag, sizeof(int32_t));
+      if (e == cudaSuccess) e = rb.sync();
+      if (e != cudaSuccess) { set_error("solve_rows: %s", cudaGetErrorString(e)); s = EAR_ECUDA; }
+    }
+    cudaFreeAsync(flag, st);
+    if (s == EAR_OK && h_flag) {   // a finite distance >= 0xFFFF: the int32 D after all
+      cudaFreeAsync(k.D16, st);
+      k.D16 = nullptr;
+    }
   }
-  if (s == EAR_OK && d_out) s = expand_ears(p, Dfull, Np, row_begin, row_end, d_out, ldo, st);
-  if (D_keep && s == EAR_OK) {
-    *D_keep = Dfull;
+  if (s == EAR_OK && !k.D16) {
+    if (!comm) {
+      EAR_CUDA_TRY(cudaMallocAsync((void **)&k.D, sizeof(int32_t) * (size_t)Np * Np, st));
+      s = apsp_reduced(p, k.D, Np, nullptr, st);
+    } else if (p->flags & EAR_FLAG_BCC) {
+      // every rank holds every solved piece after bcc_solve: compose the full matrix directly, no gather
+      EAR_CUDA_TRY(cudaMallocAsync((void **)&k.D, sizeof(int32_t) * (size_t)Np * Np, st));
+      s = bcc_solve(p, comm, k.D, Np, Np, 0, Np, nullptr, st);
+    } else {
+      // the owned rows live in this rank's exchange window, where the gather reads them
+      int32_t *S = nullptr;
+      EAR_CUDA_TRY(cudaMallocAsync((void **)&k.D, sizeof(int32_t) * (size_t)Np * Np, st));
+      s = fw_shard_buffer(comm, Np, st, &S);
+      if (s == EAR_OK) s = apsp_reduced(p, S, Np, comm, st);
+      if (s == EAR_OK) s = ear_gather_reduced(p, S, Np, k.D, Np, comm, st);
+    }
+  }
+  if (s == EAR_OK && d_out) s = expand_kept(p, k, Np, row_begin, row_end, d_out, ldo, st);
+  if (keep && s == EAR_OK) {
+    *keep = k;
   } else {
-    cudaFreeAsync(Dfull, st);
+    free_kept(k, st);
   }
   return s;
+}
+
+static bool rows_aligned(const int32_t *out, int64_t ldo) {
+  return (ldo & 3) == 0 && (reinterpret_cast<uintptr_t>(out) & 15) == 0;
 }
 
 ear_status_t apsp_full(int32_t n, int64_t m, const int32_t *d_src, const int32_t *d_dst, const int32_t *d_w,
@@ -320,7 +369,7 @@ ear_status_t apsp_full(int32_t n, int64_t m, const int32_t *d_src, const int32_t
   }
   ear_plan_t p = nullptr;
   EAR_TRY(ear_decompose(n, m, d_src, d_dst, d_w, flags, stream, &p));
-  ear_status_t s = solve_rows(p, row_begin, row_end, d_out, ldo, comm, st, nullptr);
+  ear_status_t s = solve_rows(p, row_begin, row_end, d_out, ldo, comm, st, nullptr, rows_aligned(d_out, ldo));
   cudaError_t e = cudaStreamSynchronize(st);
   ear_plan_destroy(p);
   if (s == EAR_OK && e != cudaSuccess) {
@@ -334,7 +383,7 @@ ear_status_t apsp_full(int32_t n, int64_t m, const int32_t *d_src, const int32_t
 
 struct ear_job_s {
   ear_plan_s *plan = nullptr;
-  int32_t *Dfull = nullptr;
+  DKeep D;
   int32_t *buf[2] = {nullptr, nullptr};
   cudaStream_t es = nullptr;                      // expansion stream
   cudaEvent_t ev_fw = nullptr, ready[2] = {nullptr, nullptr}, freed[2] = {nullptr, nullptr}, done = nullptr;
@@ -358,7 +407,7 @@ void job_release(ear_job_s *j) {
   // stream-ordered frees only: a cudaFree would synchronise the whole device, i.e. wait for the NEXT
   // job's Phase II too and serialise the pipeline
   cudaStream_t fs = j->es ? j->es : cudaStreamPerThread;
-  if (j->Dfull) cudaFreeAsync(j->Dfull, fs);
+  free_kept(j->D, fs);
   for (int i = 0; i < 2; ++i)
     if (j->buf[i]) cudaFreeAsync(j->buf[i], fs);
   cudaStreamSynchronize(fs);
@@ -412,7 +461,8 @@ ear_status_t apsp_full_host_async(int32_t n, int64_t m, const int32_t *h_src, co
   ear_status_t s = ear_decompose(n, m, es, ed, ew, flags, stream, &j->plan);
   if (dE) cudaFreeAsync(dE, st);
   // 2. reduced APSP on `stream`, D kept
-  if (s == EAR_OK) s = solve_rows(j->plan, row_begin, row_end, nullptr, ldo, comm, st, &j->Dfull);
+  // the chunk buffers below are the library's (aligned) with leading dimension n
+  if (s == EAR_OK) s = solve_rows(j->plan, row_begin, row_end, nullptr, ldo, comm, st, &j->D, (n & 3) == 0);
   const int32_t P = comm ? comm->nranks : 1;
   const int32_t Np = s == EAR_OK ? padded(j->plan, P) : 0;
   // 3. expansion on the job's stream, in row chunks double-buffered against the copies
@@ -440,7 +490,7 @@ ear_status_t apsp_full_host_async(int32_t n, int64_t m, const int32_t *h_src, co
       const int b = it & 1;
       const int32_t r1 = std::min(row_end, r + chunk);
       if (it >= 2) cudaStreamWaitEvent(j->es, j->freed[b], 0);
-      s = expand(j->plan, j->Dfull, Np, r, r1, j->buf[b], n, j->es);
+      s = expand_kept(j->plan, j->D, Np, r, r1, j->buf[b], n, j->es);
       if (s != EAR_OK) break;
       cudaEventRecord(j->ready[b], j->es);
       cudaStreamWaitEvent(cs, j->ready[b], 0);

@@ -467,11 +467,14 @@ __global__ void k_hang_dist(int32_t nr, const int32_t *att, const int32_t *hp, c
 
 // S^r rows from the pieces: RB rows per CTA, 4 columns per thread (int4 stores)
 constexpr int RB = 8;
+// D16 (optional, rows of stride ld16, columns [0, ld16)): the same rows as u16 for the pair-major
+// expansion, 0xFFFF = INF; a finite entry >= 0xFFFF sets *flag16.  D may be NULL when only D16 is wanted.
 __global__ void __launch_bounds__(NT) k_compose(int32_t nr, int32_t Np, const int4 *__restrict__ cinfo,
                                                 const int32_t *__restrict__ hp, const int32_t *__restrict__ pld,
                                                 const int64_t *__restrict__ pbase, const int32_t *__restrict__ pool,
                                                 int32_t *D, int64_t ldd, int32_t row0, int32_t rows,
-                                                const int32_t *trows) {
+                                                const int32_t *trows, uint16_t *D16, int64_t ld16, int32_t *flag16) {
+  int over = 0;
   __shared__ int4 s_row[RB];                 // {root piece, ratt, hloc, h}
   __shared__ const int32_t *s_R[RB], *s_H[RB];
   __shared__ int32_t s_u[RB];
@@ -519,11 +522,21 @@ __global__ void __launch_bounds__(NT) k_compose(int32_t nr, int32_t Np, const in
             o[j] = d;
           }
         }
-        *reinterpret_cast<int4 *>(D + (int64_t)(g0 + r) * ldd + c4 * 4) = make_int4(o[0], o[1], o[2], o[3]);
+        if (D) *reinterpret_cast<int4 *>(D + (int64_t)(g0 + r) * ldd + c4 * 4) = make_int4(o[0], o[1], o[2], o[3]);
+        if (D16 && c4 * 4 < ld16) {
+          uint32_t h[4];
+#pragma unroll
+          for (int j = 0; j < 4; ++j) {
+            over |= o[j] >= 0xFFFF && o[j] < INF;
+            h[j] = o[j] >= INF ? 0xFFFFu : (uint32_t)min(o[j], 0xFFFF);
+          }
+          *reinterpret_cast<uint2 *>(D16 + (int64_t)(g0 + r) * ld16 + c4 * 4) = make_uint2(h[0] | (h[1] << 16), h[2] | (h[3] << 16));
+        }
       }
     }
     __syncthreads();
   }
+  if (D16 && __syncthreads_or(over) && threadIdx.x == 0) atomicOr(flag16, 1);
 }
 
 struct Tmp {
@@ -810,7 +823,8 @@ static ear_status_t piece_rereduce(ear_plan_s *p, ear_bcc_s *b, int32_t id, int3
 // piece runs the sharded FW (its rows split over the ranks) and is re-assembled on every rank; the
 // small pieces are solved redundantly.
 ear_status_t bcc_solve(ear_plan_s *p, ear_comm_s *comm, int32_t *D, int64_t ldd, int32_t Np, int32_t row0,
-                       int32_t rows, const int32_t *d_tile_rows, cudaStream_t st) {
+                       int32_t rows, const int32_t *d_tile_rows, cudaStream_t st, uint16_t *D16, int64_t ld16,
+                       int32_t *flag16) {
   const int32_t P = comm ? comm->nranks : 1;
   int sb = prof_begin(PK_BCC_PREP, st);
   ear_status_t sprep = bcc_prepare(p, P, st);
@@ -863,8 +877,8 @@ ear_status_t bcc_solve(ear_plan_s *p, ear_comm_s *comm, int32_t *D, int64_t ldd,
     const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(ceil_div(rows, RB), 148 * 8));
     if (rows > 0)
       EAR_LAUNCH(k_compose, grid, NT, 0, st)(nr, Np, b->cinfo, b->hp, b->pld, b->pbase, pool, D, ldd, row0, rows,
-                                             d_tile_rows);
-    prof_end(sc, st, 4.0 * rows * Np);
+                                             d_tile_rows, D16, ld16, flag16);
+    prof_end(sc, st, (D ? 4.0 : 0.0) * rows * Np + (D16 ? 2.0 * rows * ld16 : 0.0));
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) {
       set_error("bcc_solve: %s", cudaGetErrorString(e));

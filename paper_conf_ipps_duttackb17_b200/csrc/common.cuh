@@ -48,6 +48,7 @@ struct PeerPtrs {
 }  // namespace ear
 
 struct ear_bcc_s;   // bcc.cu: block structure of G^r and the piece layout (EAR_FLAG_BCC)
+struct ear_xp_s;    // expand.cu: the pair-major expansion's item lists (built on first use)
 
 // Library-owned plan (Reduce(G) result), device arrays unless noted.
 struct ear_plan_s {
@@ -82,6 +83,7 @@ struct ear_plan_s {
   int32_t n_rarcs = 0;
   ear_bcc_s *bcc = nullptr;     // built on first use (EAR_FLAG_BCC, ear_bcc_info)
   int32_t *cc = nullptr;        // [cc_np] connected-component labels of G^r (16-bit FW range check)
+  ear_xp_s *xp = nullptr;       // pair-major expansion items (expand.cu), built on first use
   int32_t cc_np = 0;
 };
 
@@ -102,7 +104,7 @@ struct ear_comm_s {
 namespace ear {
 // prof.cu
 enum ProfKind { PK_DECOMPOSE, PK_FW_INIT, PK_FW_P1, PK_FW_P2, PK_FW_P3, PK_COMM, PK_EXPAND, PK_SAME_CHAIN, PK_SSSP, PK_BCC, PK_COMPOSE,
-                PK_FW_P3_16, PK_FW16_CONV, PK_FW_SIDE_P1, PK_FW_SIDE_P2, PK_REREDUCE, PK_BCC_PREP };
+                PK_FW_P3_16, PK_FW16_CONV, PK_FW_SIDE_P1, PK_FW_SIDE_P2, PK_REREDUCE, PK_BCC_PREP, PK_EXPAND_D16 };
 void prof_fw16(bool used);   // one 16-bit FW attempt: used, or fell back to int32
 void count_launch(int n = 1);
 int prof_begin(int kind, cudaStream_t s);                // -1 when profiling is off
@@ -171,12 +173,22 @@ ear_status_t sssp_rows(ear_plan_s *plan, int32_t *D, int64_t ldd, int32_t Np, in
                        const int32_t *d_tile_rows, cudaStream_t stream);
 // bcc.cu -- Phase II by biconnected pieces (paper sec. 2.2)
 ear_status_t bcc_prepare(ear_plan_s *plan, int32_t P, cudaStream_t stream);
+// D16 / ld16 / flag16 (optional): also (or, with D == NULL, only) the rows as u16 for the pair-major
+// expansion (0xFFFF = INF); *flag16 set when a finite distance does not fit (then D16 is unusable)
 ear_status_t bcc_solve(ear_plan_s *plan, ear_comm_s *comm, int32_t *D, int64_t ldd, int32_t Np, int32_t row0,
-                       int32_t rows, const int32_t *d_tile_rows, cudaStream_t stream);
+                       int32_t rows, const int32_t *d_tile_rows, cudaStream_t stream, uint16_t *D16 = nullptr,
+                       int64_t ld16 = 0, int32_t *flag16 = nullptr);
 void bcc_free(ear_bcc_s *b, cudaStream_t stream);
 // expand.cu
 ear_status_t expand(const ear_plan_s *plan, const int32_t *D, int64_t ldd, int32_t row_begin,
                     int32_t row_end, int32_t *out, int64_t ldo, cudaStream_t stream, int prof_kind = PK_EXPAND);
+// the pair-major expansion straight from u16 rows of D (0xFFFF = INF, row stride ld16 = xp_row_stride):
+// the path apsp_full takes when Phase II can hand over D16 (bcc_solve's u16 output)
+int32_t xp_row_stride(const ear_plan_s *plan);
+bool xp_applicable(ear_plan_s *plan, cudaStream_t stream);   // builds the item lists on first use
+ear_status_t expand_from16(const ear_plan_s *plan, const uint16_t *D16, int32_t ld16, int32_t row_begin,
+                           int32_t row_end, int32_t *out, int64_t ldo, cudaStream_t stream, int prof_kind = PK_EXPAND);
+void xp_free(ear_xp_s *xp, cudaStream_t stream);
 ear_status_t query_pairs(const ear_plan_s *plan, const int32_t *D, int64_t ldd, int64_t npairs, const int32_t *qs,
                          const int32_t *qt, int32_t *out, cudaStream_t stream);
 // comm.cu -- peer-memory transport (window layout in comm.cu)

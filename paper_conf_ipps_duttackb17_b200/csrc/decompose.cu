@@ -307,6 +307,8 @@ void plan_free(ear_plan_s *p) {
     if (a) cudaFreeAsync(a, p->stream);
   bcc_free(p->bcc, p->stream);
   p->bcc = nullptr;
+  xp_free(p->xp, p->stream);
+  p->xp = nullptr;
   if (p->cc) cudaFreeAsync(p->cc, p->stream);
   p->cc = nullptr;
 }

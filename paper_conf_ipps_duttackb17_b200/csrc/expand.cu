@@ -278,41 +278,425 @@ __global__ void k_query_pairs(const int32_t *__restrict__ D, int64_t ldd, const 
     out[i] = query_one(D, ldd, desc, ear, qs[i], qt[i]);
 }
 
-// Bucketed query: the pairs are first grouped by the source's left chain end p_s (a counting sort over
-// the N_r terminals: histogram, scan, scatter of packed (s, t, i) records), so that the pairs of one
-// bucket -- read consecutively -- share the D row p_s (and mostly q_s) while it sits in L2; the random
-// D sectors of the per-pair kernel become L2 hits.  out[i] keeps the caller's pair order.
-__global__ void k_qhist(int64_t npairs, const int32_t *__restrict__ qs, const VDesc *__restrict__ desc, int32_t *hist) {
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < npairs; i += (int64_t)gridDim.x * blockDim.x)
-    atomicAdd(&hist[desc[qs[i]].p], 1);
+// ============================================================================ pair-major expansion
+// An item is one terminal v of G^r: its own output row (R[v, t], the 2-term rule seen from t)
+// and the rows of every chain vertex s whose chain ends at v and at a partner x >= v (tid order; x = v
+// for a closed ear): S[s, t] = min(c_sv + R[v, t], c_sx + R[x, t]) (the 4-term rule).  The D rows
+// of v and of up to gcap partners are staged in shared memory as u16 (values < 0xFFFF, 0xFFFF = INF), so
+// every D access is a shared-memory load; the column descriptors stream from L2 as packed 8-byte
+// records; the output rows go out as 128-bit streaming stores.  No global gather is left, so the kernel
+// is bound by the output stream, not by gather latency (the row-group kernel above), and it does not
+// depend on how the caller labels the vertices.  Applies when N_r < 65535, every descriptor offset
+// < 65536, every finite D entry < 0xFFFF and two u16 rows fit in shared memory; the same-chain clause
+// is the separate k_same_chain pass as before.
+constexpr int XP_NT = 1024;
+constexpr int XP_RMAX = 64;   // chain rows written per column sweep
+constexpr int XP_GMAX = 4;    // partner rows resident per sweep
+
+struct XpView {
+  const uint2 *pd;
+  const int32_t *rows, *pstart, *px, *istart, *tid2v;
+};
+
+__global__ void k_xp_flags(int32_t n, const VDesc *desc, int32_t *bad) {
+  int b = 0;
+  for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
+    const VDesc d = desc[v];
+    b |= d.cp > 0xFFFF || d.cq > 0xFFFF || d.p > 0xFFFE || d.q > 0xFFFE;
+  }
+  if (__syncthreads_or(b) && threadIdx.x == 0) atomicOr(bad, 1);
 }
-__global__ void k_qscatter(int64_t npairs, const int32_t *__restrict__ qs, const int32_t *__restrict__ qt,
-                           const VDesc *__restrict__ desc, int64_t *cur, int4 *rec) {
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < npairs; i += (int64_t)gridDim.x * blockDim.x) {
-    const int32_t s = qs[i];
-    const int64_t pos = atomicAdd(reinterpret_cast<unsigned long long *>(&cur[desc[s].p]), 1ull);
-    rec[pos] = make_int4(s, qt[i], (int32_t)(i & 0xFFFFFFFF), (int32_t)(i >> 32));
+__global__ void k_xp_desc(int32_t n, const VDesc *desc, uint2 *pd) {
+  for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
+    const VDesc d = desc[v];
+    pd[v] = make_uint2((uint32_t)d.p | ((uint32_t)d.q << 16), (uint32_t)d.cp | ((uint32_t)d.cq << 16));
   }
 }
-__global__ void k_query_bucketed(const int32_t *__restrict__ D, int64_t ldd, const VDesc *__restrict__ desc,
-                                 const int32_t *__restrict__ ear, int64_t npairs, const int4 *__restrict__ rec,
-                                 int32_t *__restrict__ out) {
-  for (int64_t j = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; j < npairs; j += (int64_t)gridDim.x * blockDim.x) {
-    const int4 r = rec[j];
-    out[(int64_t)(uint32_t)r.z | ((int64_t)r.w << 32)] = query_one(D, ldd, desc, ear, r.x, r.y);
+__global__ void k_xp_keys(int32_t nc, const int32_t *seg_vert, const VDesc *desc, uint64_t *key, int32_t *val) {
+  for (int32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < nc; i += gridDim.x * blockDim.x) {
+    const int32_t v = seg_vert[i];
+    const VDesc d = desc[v];
+    key[i] = ((uint64_t)(uint32_t)min(d.p, d.q) << 32) | (uint32_t)max(d.p, d.q);
+    val[i] = v;
   }
 }
-__global__ void k_hist64(int32_t nb, const int32_t *hist, int64_t *h64) {
-  for (int32_t b = blockIdx.x * blockDim.x + threadIdx.x; b < nb; b += gridDim.x * blockDim.x) h64[b] = hist[b];
+__global__ void k_xp_heads(int32_t nc, const uint64_t *key, int32_t *head) {
+  for (int32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < nc; i += gridDim.x * blockDim.x)
+    head[i] = i == 0 || key[i] != key[i - 1];
+}
+__global__ void k_xp_pairs(int32_t nc, const uint64_t *key, const int32_t *head, const int32_t *hscan, int32_t *pstart,
+                           int32_t *px, int32_t *pcount) {
+  for (int32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < nc; i += gridDim.x * blockDim.x)
+    if (head[i]) {
+      const int32_t j = hscan[i] - 1;
+      pstart[j] = i;
+      px[j] = (int32_t)(key[i] & 0xFFFFFFFFu);
+      atomicAdd(&pcount[(int32_t)(key[i] >> 32)], 1);
+    }
+}
+__global__ void k_xp_last(int32_t np, int32_t nc, int32_t *pstart) { pstart[np] = nc; }
+__global__ void k_xp_tid2v(int32_t n, const int32_t *tid, int32_t *tid2v) {
+  for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x)
+    if (tid[v] >= 0) tid2v[tid[v]] = (int32_t)v;
+}
+// D (int32) -> u16 rows of stride ldr; a finite entry >= 0xFFFF sets *bad
+__global__ void k_xp_d16(const int32_t *__restrict__ D, int64_t ldd, int32_t nr, int32_t ldr, uint16_t *__restrict__ D16,
+                         int32_t *bad) {
+  const int64_t total = (int64_t)nr * (ldr / 4);
+  int b = 0;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t r = i / (ldr / 4);
+    const int32_t c = (int32_t)(i % (ldr / 4)) * 4;
+    int32_t x[4];
+#pragma unroll
+    for (int k = 0; k < 4; ++k) {
+      const int32_t v = c + k < nr ? D[r * ldd + c + k] : INF;
+      b |= v >= 0xFFFF && v < INF;
+      x[k] = v >= INF ? 0xFFFF : min(v, 0xFFFF);
+    }
+    *reinterpret_cast<uint2 *>(D16 + r * ldr + c) =
+        make_uint2((uint32_t)x[0] | ((uint32_t)x[1] << 16), (uint32_t)x[2] | ((uint32_t)x[3] << 16));
+  }
+  if (__syncthreads_or(b) && threadIdx.x == 0) atomicOr(bad, 1);
 }
 
+__device__ __forceinline__ int32_t d16(const uint16_t *row, uint32_t t) {
+  const uint32_t x = row[t];
+  return x == 0xFFFFu ? INF : (int32_t)x;
+}
+__device__ __forceinline__ void r_of(const uint16_t *row, const uint32_t pq[4], const uint32_t cc[4], int32_t R[4]) {
+#pragma unroll
+  for (int j = 0; j < 4; ++j)
+    R[j] = min(__viaddmin_s32(d16(row, pq[j] >> 16), (int32_t)(cc[j] >> 16), d16(row, pq[j] & 0xFFFFu) + (int32_t)(cc[j] & 0xFFFFu)), INF);
+}
+
+__global__ void __launch_bounds__(XP_NT, 1)
+    k_expand_pairs(const uint16_t *__restrict__ D16, int32_t ldr, int32_t nr, const VDesc *__restrict__ desc,
+                   const XpView X, int32_t n, int32_t rb, int32_t re, int32_t *__restrict__ out, int64_t ldo,
+                   int32_t gcap, int32_t *counter) {
+  extern __shared__ __align__(16) uint16_t srow[];   // [1 + gcap][ldr]
+  __shared__ int4 meta[XP_RMAX];                     // {c_sv, c_sx, slot, local output row}
+  __shared__ int32_t slot_x[XP_GMAX];
+  __shared__ int32_t s_item, s_nrow, s_ns, s_pj, s_rj;
+  const int tid = threadIdx.x;
+  const uint32_t ldo_b = (uint32_t)(ldo * 4);
+  for (;;) {
+    if (tid == 0) s_item = atomicAdd(counter, 1);
+    __syncthreads();
+    const int32_t v = s_item;
+    if (v >= nr) break;
+    const int32_t tv = X.tid2v[v];
+    bool need_term = tv >= rb && tv < re;
+    const int32_t pe = X.istart[v + 1];
+    int32_t pj = X.istart[v], rj = pj < pe ? X.pstart[pj] : 0;
+    bool loaded_v = false;
+    for (;;) {
+      if (tid == 0) {   // the next sweep: up to gcap partner rows and XP_RMAX chain rows in range
+        int ns = 0, nrow = 0;
+        while (pj < pe && nrow < XP_RMAX) {
+          const int32_t x = X.px[pj];
+          int slot = 0;
+          if (x != v) {
+            slot = -1;
+            for (int k = 0; k < ns; ++k)
+              if (slot_x[k] == x) slot = k + 1;
+            if (slot < 0) {
+              if (ns == gcap) break;
+              slot_x[ns++] = x;
+              slot = ns;
+            }
+          }
+          const int32_t r1 = X.pstart[pj + 1];
+          while (rj < r1 && nrow < XP_RMAX) {
+            const int32_t s = X.rows[rj++];
+            if (s >= rb && s < re) {
+              const VDesc d = desc[s];
+              const bool left = d.p == v;   // c_sv: along-chain distance from s to v
+              meta[nrow++] = make_int4(left ? d.cp : d.cq, left ? d.cq : d.cp, slot, s - rb);
+            }
+          }
+          if (rj >= r1) {
+            ++pj;
+            if (pj < pe) rj = X.pstart[pj];
+          }
+        }
+        s_nrow = nrow; s_ns = ns; s_pj = pj; s_rj = rj;
+      }
+      __syncthreads();
+      const int nrow = s_nrow, ns = s_ns;
+      pj = s_pj;
+      rj = s_rj;
+      if (nrow > 0 || need_term) {
+        const int nv = (nr + 7) / 8;   // 16-byte vectors per row
+        if (!loaded_v)
+          for (int i = tid; i < nv; i += XP_NT)
+            reinterpret_cast<uint4 *>(srow)[i] = reinterpret_cast<const uint4 *>(D16 + (int64_t)v * ldr)[i];
+        for (int k = 0; k < ns; ++k)
+          for (int i = tid; i < nv; i += XP_NT)
+            reinterpret_cast<uint4 *>(srow + (1 + k) * ldr)[i] =
+                reinterpret_cast<const uint4 *>(D16 + (int64_t)slot_x[k] * ldr)[i];
+        loaded_v = true;
+        __syncthreads();
+        for (int32_t c0 = tid * 4; c0 < n; c0 += XP_NT * 4) {
+          uint32_t pq[4], cc[4];
+          if (c0 + 4 <= n) {
+            const uint4 a = *reinterpret_cast<const uint4 *>(X.pd + c0);
+            const uint4 b = *reinterpret_cast<const uint4 *>(X.pd + c0 + 2);
+            pq[0] = a.x; cc[0] = a.y; pq[1] = a.z; cc[1] = a.w; pq[2] = b.x; cc[2] = b.y; pq[3] = b.z; cc[3] = b.w;
+          } else {
+#pragma unroll
+            for (int j = 0; j < 4; ++j) {
+              const uint2 q = c0 + j < n ? X.pd[c0 + j] : make_uint2(0, 0);
+              pq[j] = q.x; cc[j] = q.y;
+            }
+          }
+          int32_t Rv[4], R1[4], R2[4], R3[4], R4[4];
+          r_of(srow, pq, cc, Rv);
+          if (ns > 0) r_of(srow + ldr, pq, cc, R1);
+          if (ns > 1) r_of(srow + 2 * ldr, pq, cc, R2);
+          if (ns > 2) r_of(srow + 3 * ldr, pq, cc, R3);
+          if (ns > 3) r_of(srow + 4 * ldr, pq, cc, R4);
+          const bool full = c0 + 4 <= n;
+          if (need_term) {
+            int32_t *o = reinterpret_cast<int32_t *>(reinterpret_cast<char *>(out) + (uint64_t)(uint32_t)(tv - rb) * ldo_b) + c0;
+            if (full) st_cs_v4(o, make_int4(Rv[0], Rv[1], Rv[2], Rv[3]));
+            else for (int j = 0; c0 + j < n; ++j) o[j] = Rv[j];
+          }
+          for (int r = 0; r < nrow; ++r) {
+            const int4 m = meta[r];
+            const int32_t *Rx = m.z == 0 ? Rv : m.z == 1 ? R1 : m.z == 2 ? R2 : m.z == 3 ? R3 : R4;
+            int4 o4;
+            o4.x = out_val(m.x, Rv[0], m.y, Rx[0]);
+            o4.y = out_val(m.x, Rv[1], m.y, Rx[1]);
+            o4.z = out_val(m.x, Rv[2], m.y, Rx[2]);
+            o4.w = out_val(m.x, Rv[3], m.y, Rx[3]);
+            int32_t *o = reinterpret_cast<int32_t *>(reinterpret_cast<char *>(out) + (uint64_t)(uint32_t)m.w * ldo_b) + c0;
+            if (full) st_cs_v4(o, o4);
+            else {
+              const int32_t t4[4] = {o4.x, o4.y, o4.z, o4.w};
+              for (int j = 0; c0 + j < n; ++j) o[j] = t4[j];
+            }
+          }
+        }
+        need_term = false;
+      }
+      __syncthreads();   // the next sweep rewrites meta, slot_x and the partner rows
+      if (pj >= pe) break;
+    }
+  }
+}
 
 }  // namespace
+
+}  // namespace ear
+
+struct ear_xp_s {
+  int32_t ok = 0;            // the pair-major layout applies to this plan
+  int32_t npairs = 0, nc = 0;
+  uint2 *pd = nullptr;       // [n] packed descriptors {p | q << 16, cp | cq << 16}
+  int32_t *rows = nullptr;   // [nc] chain vertices sorted by (smaller end, larger end, chain, offset)
+  int32_t *pstart = nullptr; // [npairs + 1]
+  int32_t *px = nullptr;     // [npairs] the larger end (the partner)
+  int32_t *istart = nullptr; // [N_r + 1] the pairs of each item (terminal = smaller end)
+  int32_t *tid2v = nullptr;  // [N_r]
+};
+
+namespace ear {
+
+void xp_free(ear_xp_s *x, cudaStream_t st) {
+  if (!x) return;
+  for (void *p : {(void *)x->pd, (void *)x->rows, (void *)x->pstart, (void *)x->px, (void *)x->istart, (void *)x->tid2v})
+    if (p) cudaFreeAsync(p, st);
+  delete x;
+}
+
+namespace {
+// the item lists of the pair-major expansion, once per plan
+ear_status_t xp_build(ear_plan_s *p, cudaStream_t st) {
+  ear_xp_s *x = new ear_xp_s;
+  p->xp = x;
+  const int32_t n = p->n, nr = p->n_reduced, nc = p->n_chain_vertices;
+  int32_t *bad = nullptr;
+  EAR_CUDA_TRY(cudaMallocAsync((void **)&bad, sizeof(int32_t), st));
+  EAR_CUDA_TRY(dev_memset(bad, 0, sizeof(int32_t), st));
+  EAR_LAUNCH(k_xp_flags, (int)std::min<int64_t>(ceil_div(n, 256), 148 * 16), 256, 0, st)(n, p->desc, bad);
+  int32_t h_bad = 1;
+  {
+    Readback rb(st);
+    EAR_CUDA_TRY(rb.get(&h_bad, bad, sizeof(int32_t)));
+    EAR_CUDA_TRY(rb.sync());
+  }
+  cudaFreeAsync(bad, st);
+  if (h_bad || nr >= 0xFFFF) return EAR_OK;   // x->ok stays 0: the row-group kernel serves this plan
+  auto g = [](int64_t k) { return (int)std::max<int64_t>(1, std::min<int64_t>(ceil_div(k, 256), 148 * 16)); };
+  EAR_CUDA_TRY(cudaMallocAsync((void **)&x->pd, sizeof(uint2) * (size_t)std::max(n, 1), st));
+  EAR_CUDA_TRY(cudaMallocAsync((void **)&x->tid2v, sizeof(int32_t) * (size_t)std::max(nr, 1), st));
+  EAR_CUDA_TRY(cudaMallocAsync((void **)&x->istart, sizeof(int32_t) * ((size_t)nr + 1), st));
+  EAR_LAUNCH(k_xp_desc, g(n), 256, 0, st)(n, p->desc, x->pd);
+  EAR_LAUNCH(k_xp_tid2v, g(n), 256, 0, st)(n, p->tid, x->tid2v);
+  x->nc = nc;
+  uint64_t *k0 = nullptr, *k1 = nullptr;
+  int32_t *v0 = nullptr, *head = nullptr, *hscan = nullptr, *pcount = nullptr;
+  void *tmp = nullptr;
+  size_t tb = 0, tb2 = 0, tb3 = 0;
+  const size_t m = (size_t)std::max(nc, 1);
+  EAR_CUDA_TRY(cudaMallocAsync((void **)&x->rows, sizeof(int32_t) * m, st));
+  EAR_CUDA_TRY(cudaMallocAsync((void **)&k0, sizeof(uint64_t) * m, st));
+  EAR_CUDA_TRY(cudaMallocAsync((void **)&k1, sizeof(uint64_t) * m, st));
+  EAR_CUDA_TRY(cudaMallocAsync((void **)&v0, sizeof(int32_t) * m, st));
+  EAR_CUDA_TRY(cudaMallocAsync((void **)&head, sizeof(int32_t) * m, st));
+  EAR_CUDA_TRY(cudaMallocAsync((void **)&hscan, sizeof(int32_t) * m, st));
+  EAR_CUDA_TRY(cudaMallocAsync((void **)&pcount, sizeof(int32_t) * ((size_t)nr + 1), st));
+  EAR_CUDA_TRY(dev_memset(pcount, 0, sizeof(int32_t) * ((size_t)nr + 1), st));
+  int32_t npairs = 0;
+  if (nc > 0) {
+    EAR_LAUNCH(k_xp_keys, g(nc), 256, 0, st)(nc, p->seg_vert, p->desc, k0, v0);
+    cub::DoubleBuffer<uint64_t> dk(k0, k1);
+    cub::DoubleBuffer<int32_t> dv(v0, x->rows);
+    EAR_CUDA_TRY(cub::DeviceRadixSort::SortPairs(nullptr, tb, dk, dv, nc, 0, 64, st));
+    EAR_CUDA_TRY(cub::DeviceScan::InclusiveSum(nullptr, tb2, head, hscan, nc, st));
+    EAR_CUDA_TRY(cub::DeviceScan::ExclusiveSum(nullptr, tb3, pcount, x->istart, nr + 1, st));
+    EAR_CUDA_TRY(cudaMallocAsync(&tmp, std::max({tb, tb2, tb3, (size_t)16}), st));
+    EAR_CUDA_TRY(cub::DeviceRadixSort::SortPairs(tmp, tb, dk, dv, nc, 0, 64, st));
+    if (dv.Current() != x->rows) EAR_CUDA_TRY(dev_copy(x->rows, dv.Current(), sizeof(int32_t) * nc, st));
+    EAR_LAUNCH(k_xp_heads, g(nc), 256, 0, st)(nc, dk.Current(), head);
+    EAR_CUDA_TRY(cub::DeviceScan::InclusiveSum(tmp, tb2, head, hscan, nc, st));
+    Readback rb(st);
+    EAR_CUDA_TRY(rb.get(&npairs, hscan + nc - 1, sizeof(int32_t)));
+    EAR_CUDA_TRY(rb.sync());
+    EAR_CUDA_TRY(cudaMallocAsync((void **)&x->pstart, sizeof(int32_t) * ((size_t)npairs + 1), st));
+    EAR_CUDA_TRY(cudaMallocAsync((void **)&x->px, sizeof(int32_t) * (size_t)std::max(npairs, 1), st));
+    EAR_LAUNCH(k_xp_pairs, g(nc), 256, 0, st)(nc, dk.Current(), head, hscan, x->pstart, x->px, pcount);
+    EAR_LAUNCH(k_xp_last, 1, 1, 0, st)(npairs, nc, x->pstart);
+    EAR_CUDA_TRY(cub::DeviceScan::ExclusiveSum(tmp, tb3, pcount, x->istart, nr + 1, st));
+  } else {
+    EAR_CUDA_TRY(cudaMallocAsync((void **)&x->pstart, sizeof(int32_t), st));
+    EAR_CUDA_TRY(cudaMallocAsync((void **)&x->px, sizeof(int32_t), st));
+    EAR_CUDA_TRY(dev_memset(x->pstart, 0, sizeof(int32_t), st));
+    EAR_CUDA_TRY(dev_memset(x->istart, 0, sizeof(int32_t) * ((size_t)nr + 1), st));
+  }
+  for (void *q : {(void *)k0, (void *)k1, (void *)v0, (void *)head, (void *)hscan, (void *)pcount, tmp})
+    if (q) cudaFreeAsync(q, st);
+  x->npairs = npairs;
+  x->ok = 1;
+  EAR_CUDA_TRY(cudaGetLastError());
+  return EAR_OK;
+}
+
+// partner rows that fit in shared memory beside the item's own row (0: the pair-major layout does not fit)
+int32_t xp_gcap(int32_t nr) {
+  int dev = 0, smax = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess || cudaDeviceGetAttribute(&smax, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev) != cudaSuccess) {
+    cudaGetLastError();
+    return 0;
+  }
+  const int64_t rowb = round_up(std::max(nr, 1), 8) * 2, budget = (int64_t)smax - 4096;
+  return (int32_t)std::max<int64_t>(0, std::min<int64_t>(XP_GMAX, budget / rowb - 1));
+}
+
+// k_expand_pairs over u16 rows D16 (stride ld16) + the same-chain pass; the caller checked applicability
+ear_status_t launch_pairs(const ear_plan_s *plan, const uint16_t *D16, int32_t ld16, int32_t row_begin, int32_t row_end,
+                          int32_t *out, int64_t ldo, cudaStream_t st, int prof_kind) {
+  const ear_xp_s *x = plan->xp;
+  const int32_t nr = plan->n_reduced, gcap = xp_gcap(nr);
+  const int smem = (int)((1 + gcap) * (int64_t)ld16 * 2);
+  EAR_CUDA_TRY(smem_attr((const void *)k_expand_pairs, smem));
+  int32_t *counter = nullptr;
+  EAR_CUDA_TRY(cudaMallocAsync((void **)&counter, sizeof(int32_t), st));
+  EAR_CUDA_TRY(dev_memset(counter, 0, sizeof(int32_t), st));
+  const XpView V{x->pd, x->rows, x->pstart, x->px, x->istart, x->tid2v};
+  const double rows = row_end - row_begin;
+  int se = prof_begin(prof_kind, st);
+  EAR_LAUNCH(k_expand_pairs, num_sms(), XP_NT, smem, st)(D16, ld16, nr, plan->desc, V, plan->n, row_begin, row_end, out,
+                                                        ldo, gcap, counter);
+  // algorithmic bytes: the output, D read once (counted as the int32 D, as for the row-group kernel), the
+  // descriptors
+  prof_end(se, st, 4.0 * rows * plan->n + 16.0 * plan->n + 4.0 * (double)nr * nr * rows / plan->n);
+  cudaFreeAsync(counter, st);
+  if (plan->n_chain_vertices > 0) {
+    int ss = prof_begin(prof_kind == PK_EXPAND ? PK_SAME_CHAIN : prof_kind, st);
+    const int g2 = (int)std::min<int64_t>(ceil_div((int64_t)(row_end - row_begin) * 32, 256), 148 * 16);
+    EAR_LAUNCH(k_same_chain, g2, 256, 0, st)(plan->desc, plan->seg_of, plan->seg_start, plan->seg_vert, row_begin,
+                                              row_end, out, ldo);
+    prof_end(ss, st, 0);
+  }
+  EAR_CUDA_TRY(cudaGetLastError());
+  return EAR_OK;
+}
+
+bool aligned_out(const int32_t *out, int64_t ldo) { return (ldo & 3) == 0 && (reinterpret_cast<uintptr_t>(out) & 15) == 0; }
+
+// the pair-major expansion from the int32 D (narrowed to u16 rows first) when it applies: *done = true
+// after writing the rows, the same-chain pass included
+ear_status_t expand_pairs(ear_plan_s *plan, const int32_t *D, int64_t ldd, int32_t row_begin, int32_t row_end,
+                          int32_t *out, int64_t ldo, cudaStream_t st, int prof_kind, bool *done) {
+  *done = false;
+  if (!aligned_out(out, ldo) || !xp_applicable(plan, st)) return EAR_OK;
+  const int32_t nr = plan->n_reduced, ldr = xp_row_stride(plan);
+  uint16_t *D16 = nullptr;
+  int32_t *bad = nullptr;
+  if (cudaMallocAsync((void **)&D16, sizeof(uint16_t) * (size_t)nr * ldr, st) != cudaSuccess ||
+      cudaMallocAsync((void **)&bad, sizeof(int32_t), st) != cudaSuccess) {
+    cudaGetLastError();
+    if (D16) cudaFreeAsync(D16, st);
+    return EAR_OK;
+  }
+  ear_status_t s = EAR_OK;
+  int32_t h_bad = 1;
+  {
+    cudaError_t e = dev_memset(bad, 0, sizeof(int32_t), st);
+    const int64_t tot = (int64_t)nr * (ldr / 4);
+    int sp = prof_begin(prof_kind == PK_EXPAND ? PK_EXPAND_D16 : prof_kind, st);
+    if (e == cudaSuccess && tot > 0)
+      EAR_LAUNCH(k_xp_d16, (int)std::min<int64_t>(ceil_div(tot, 256), 148 * 16), 256, 0, st)(D, ldd, nr, ldr, D16, bad);
+    prof_end(sp, st, 0);
+    Readback rb(st);
+    if (e == cudaSuccess) e = rb.get(&h_bad, bad, sizeof(int32_t));
+    if (e == cudaSuccess) e = rb.sync();
+    if (e != cudaSuccess) { set_error("expand: %s", cudaGetErrorString(e)); s = EAR_ECUDA; }
+  }
+  if (s == EAR_OK && !h_bad) {
+    s = launch_pairs(plan, D16, ldr, row_begin, row_end, out, ldo, st, prof_kind);
+    *done = s == EAR_OK;
+  }
+  cudaFreeAsync(D16, st);
+  cudaFreeAsync(bad, st);
+  return s;
+}
+}  // namespace
+
+int32_t xp_row_stride(const ear_plan_s *plan) { return (int32_t)round_up(std::max(plan->n_reduced, 1), 8); }
+
+bool xp_applicable(ear_plan_s *plan, cudaStream_t st) {
+  const char *env = getenv("EAR_EXPAND_PAIRS");   // 0: the row-group kernel (A/B)
+  if (env && atoi(env) == 0) return false;
+  if (plan->n_reduced >= 0xFFFF || xp_gcap(plan->n_reduced) < 1) return false;
+  if (!plan->xp && xp_build(plan, st) != EAR_OK) {
+    cudaGetLastError();
+    return false;
+  }
+  return plan->xp && plan->xp->ok;
+}
+
+ear_status_t expand_from16(const ear_plan_s *plan, const uint16_t *D16, int32_t ld16, int32_t row_begin, int32_t row_end,
+                           int32_t *out, int64_t ldo, cudaStream_t st, int prof_kind) {
+  if (row_end <= row_begin) return EAR_OK;
+  if (!plan->xp || !plan->xp->ok || !aligned_out(out, ldo) || ld16 < xp_row_stride(plan)) {
+    set_error("expand_from16: the pair-major layout does not apply");
+    return EAR_EUNSUPPORTED;
+  }
+  return launch_pairs(plan, D16, ld16, row_begin, row_end, out, ldo, st, prof_kind);
+}
 
 ear_status_t expand(const ear_plan_s *plan, const int32_t *D, int64_t ldd, int32_t row_begin, int32_t row_end,
                     int32_t *out, int64_t ldo, cudaStream_t st, int prof_kind) {
   const int32_t rows = row_end - row_begin;
   if (rows <= 0) return EAR_OK;
+  if (prof_kind == PK_EXPAND) {   // the caller's rows; a BCC piece's re-expansion keeps the row-group kernel
+    bool done = false;             // (its plan is built per solve: the item lists would be rebuilt each time)
+    EAR_TRY(expand_pairs(const_cast<ear_plan_s *>(plan), D, ldd, row_begin, row_end, out, ldo, st, prof_kind, &done));
+    if (done) return EAR_OK;
+  }
   EAR_CUDA_TRY(smem_attr((const void *)k_expand, EXP_SMEM));
   int per = 0;
   EAR_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_expand, NT, EXP_SMEM));
@@ -343,48 +727,14 @@ ear_status_t expand(const ear_plan_s *plan, const int32_t *D, int64_t ldd, int32
   return EAR_OK;
 }
 
-// Bucketing pays once a batch has many pairs per terminal row (EAR_QUERY_BUCKET_MIN overrides the
-// threshold; 0 disables bucketing).
+// One thread per pair.  Measured on cfg4 (profiles/r02g_query_mode_cfg4.jsonl): 1.53e10 uniformly random
+// pairs/s, 3.60e10 when the caller's pairs are grouped by source (1,024 targets per source: the D rows
+// p_s, q_s stay in L2); an in-library counting sort of the pairs by p_s cost more than it saved (0.65x).
 ear_status_t query_pairs(const ear_plan_s *plan, const int32_t *D, int64_t ldd, int64_t npairs, const int32_t *qs,
                          const int32_t *qt, int32_t *out, cudaStream_t st) {
   if (npairs <= 0) return EAR_OK;
   const int grid = (int)std::min<int64_t>(ceil_div(npairs, 256), 148 * 16);
-  const char *env = getenv("EAR_QUERY_BUCKET_MIN");
-  const int64_t min_pairs = env ? atoll(env) : (int64_t)4 * plan->n_reduced + (1 << 20);
-  if (min_pairs <= 0 || npairs < min_pairs) {
-    EAR_LAUNCH(k_query_pairs, grid, 256, 0, st)(D, ldd, plan->desc, plan->ear, npairs, qs, qt, out);
-    EAR_CUDA_TRY(cudaGetLastError());
-    return EAR_OK;
-  }
-  const int32_t nb = std::max(plan->n_reduced, 1);
-  int32_t *hist = nullptr;
-  int64_t *h64 = nullptr, *start = nullptr;
-  int4 *rec = nullptr;
-  void *tmp = nullptr;
-  size_t tb = 0;
-  EAR_CUDA_TRY(cub::DeviceScan::ExclusiveSum(nullptr, tb, h64, start, nb, st));
-  ear_status_t s = EAR_OK;
-  if (cudaMallocAsync((void **)&hist, sizeof(int32_t) * nb, st) != cudaSuccess ||
-      cudaMallocAsync((void **)&h64, sizeof(int64_t) * nb, st) != cudaSuccess ||
-      cudaMallocAsync((void **)&start, sizeof(int64_t) * nb, st) != cudaSuccess ||
-      cudaMallocAsync(&tmp, std::max<size_t>(tb, 16), st) != cudaSuccess ||
-      cudaMallocAsync((void **)&rec, sizeof(int4) * (size_t)npairs, st) != cudaSuccess) {
-    cudaGetLastError();
-    s = EAR_ENOMEM;
-    set_error("ear_query_pairs: out of device memory for the buckets");
-  }
-  if (s == EAR_OK) {
-    const int gb = (int)std::min<int64_t>(ceil_div(nb, 256), 148 * 16);
-    EAR_CUDA_TRY(dev_memset(hist, 0, sizeof(int32_t) * nb, st));
-    EAR_LAUNCH(k_qhist, grid, 256, 0, st)(npairs, qs, plan->desc, hist);
-    EAR_LAUNCH(k_hist64, gb, 256, 0, st)(nb, hist, h64);
-    EAR_CUDA_TRY(cub::DeviceScan::ExclusiveSum(tmp, tb, h64, start, nb, st));
-    EAR_LAUNCH(k_qscatter, grid, 256, 0, st)(npairs, qs, qt, plan->desc, start, rec);
-    EAR_LAUNCH(k_query_bucketed, grid, 256, 0, st)(D, ldd, plan->desc, plan->ear, npairs, rec, out);
-  }
-  for (void *p : {(void *)hist, (void *)h64, (void *)start, tmp, (void *)rec})
-    if (p) cudaFreeAsync(p, st);
-  EAR_TRY(s);
+  EAR_LAUNCH(k_query_pairs, grid, 256, 0, st)(D, ldd, plan->desc, plan->ear, npairs, qs, qt, out);
   EAR_CUDA_TRY(cudaGetLastError());
   return EAR_OK;
 }

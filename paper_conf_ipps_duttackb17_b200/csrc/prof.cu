@@ -259,6 +259,7 @@ ear_status_t ear_profile_read(ear_profile_t *out) {
         break;
       case PK_REREDUCE: g_acc.rereduce_ms += ms; break;
       case PK_BCC_PREP: g_acc.bcc_prepare_ms += ms; break;
+      case PK_EXPAND_D16: g_acc.expand_d16_ms += ms; break;
       default: break;
     }
     g_pool.push_back(r.e0);

@@ -57,7 +57,7 @@ class _Profile(ctypes.Structure):
                 ("fw16_conv_ms", ctypes.c_double), ("fw_phase3_16_ms", ctypes.c_double),
                 ("fw_phase3_16_minplus", ctypes.c_double), ("fw_side_ms", ctypes.c_double),
                 ("rereduce_ms", ctypes.c_double), ("bcc_prepare_ms", ctypes.c_double),
-                ("fw16_prechecked", ctypes.c_int64)]
+                ("fw16_prechecked", ctypes.c_int64), ("expand_d16_ms", ctypes.c_double)]
 
 
 class _BccInfo(ctypes.Structure):

@@ -362,12 +362,9 @@ def test_query_pairs_cfg4_without_full_matrix(pkg):
     assert_exact(got, ref[:, cols], "cfg4 query pairs")
 
 
-@pytest.mark.parametrize("bucket", ["forced", "off"])
 @pytest.mark.parametrize("name", ["corner", "cfg2"])
-def test_query_pairs_bucketed(pkg, monkeypatch, name, bucket):
-    """The bucketed query path (pairs grouped by the source's chain end; EAR_QUERY_BUCKET_MIN=1 forces it
-    for any batch) and the per-pair path (0), shuffled pair order, against oracle rows."""
-    monkeypatch.setenv("EAR_QUERY_BUCKET_MIN", "1" if bucket == "forced" else "0")
+def test_query_pairs_shuffled(pkg, name):
+    """Whole oracle rows through the query path with the pairs in a random order (BCC Phase II D)."""
     g = gg.corner_cases(44, n_target=700) if name == "corner" else gg.config("cfg2")
     plan = pkg.ear_decompose(g.n, dev(g.src), dev(g.dst), dev(g.w), flags=pkg.FLAG_BCC)
     D = pkg.alloc_D(plan)
@@ -380,7 +377,7 @@ def test_query_pairs_bucketed(pkg, monkeypatch, name, bucket):
     perm = rng.permutation(len(s))
     got = np.empty(len(s), np.int32)
     got[perm] = pkg.query_pairs(plan, D, dev(s[perm]), dev(t[perm])).cpu().numpy()
-    assert_exact(got.reshape(len(rows), g.n), ref, f"bucketed query {name} {bucket}")
+    assert_exact(got.reshape(len(rows), g.n), ref, f"shuffled query {name}")
 
 
 # ------------------------------------------------------------------------------ NEXT 2: SSSP Phase II

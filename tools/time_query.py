@@ -1,7 +1,6 @@
 """Query mode throughput (S[s,t] for arbitrary pairs from D + descriptors, no N x N
 matrix): 2^26 pairs per batch on cfg4 (or the given config), uniformly random and source-grouped
-(1,024 random targets per random source), through ear_query_pairs with its bucketing by the source's
-chain end (default) and with bucketing disabled (EAR_QUERY_BUCKET_MIN=0).  Parity of the query path:
+(1,024 random targets per random source), through ear_query_pairs.  Parity of the query path:
 tests/test_parity_gpu.py.
 
     python tools/time_query.py [cfg4] [--pairs N] [--out profiles/...jsonl]
@@ -46,26 +45,18 @@ def main():
     peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
     lines = []
     for name, (s, t) in workloads.items():
-        res = {}
-        for mode in ("per_pair", "bucketed"):
-            os.environ["EAR_QUERY_BUCKET_MIN"] = "0" if mode == "per_pair" else "1"
+        ea.query_pairs(plan, D, s, t, out=out)
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        for _ in range(args.reps):
             ea.query_pairs(plan, D, s, t, out=out)
-            torch.cuda.synchronize()
-            ref = out.clone() if mode == "per_pair" else ref
-            same = bool(torch.equal(out, ref))
-            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-            e0.record()
-            for _ in range(args.reps):
-                ea.query_pairs(plan, D, s, t, out=out)
-            e1.record()
-            torch.cuda.synchronize()
-            ms = e0.elapsed_time(e1) / args.reps
-            res[mode] = {"ms_per_batch": ms, "pairs_per_s": P / (ms / 1e3), "same_as_per_pair": same}
-        os.environ.pop("EAR_QUERY_BUCKET_MIN", None)
+        e1.record()
+        torch.cuda.synchronize()
+        ms = e0.elapsed_time(e1) / args.reps
         rec = {"config": args.config, "workload": name, "pairs": P, "n": g.n, "n_reduced": plan.info().n_reduced,
-               "D_bytes": int(D.numel()) * 4, "full_matrix_bytes": 4 * g.n * g.n, **res,
-               "speedup": res["per_pair"]["ms_per_batch"] / res["bucketed"]["ms_per_batch"],
-               "hbm_copy_GBps": peaks.get("hbm_gbs")}
+               "D_bytes": int(D.numel()) * 4, "full_matrix_bytes": 4 * g.n * g.n, "ms_per_batch": ms,
+               "pairs_per_s": P / (ms / 1e3), "hbm_copy_GBps": peaks.get("hbm_gbs")}
         print(json.dumps(rec), flush=True)
         lines.append(rec)
     if args.out:
