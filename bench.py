@@ -334,9 +334,9 @@ def run_ours(args, rank, world, local_rank):
     p3_ms = prof["fw_phase3_ms"]
     ach = prof["fw_phase3_minplus"] / (p3_ms / 1e3) / 1e12 if p3_ms > 0 else 0.0
     n_p3 = max(prof["fw_phase3_launches"], 1)
-    roofline = {"bound": "alu", "kernel": "k_fw_tiles (FW phase 3)", "achieved": ach, "peak": peak_alu,
+    roofline = {"bound": "alu", "kernel": "k_fw_tiles<Frag32> (FW phase 3, int32)", "achieved": ach, "peak": peak_alu,
                 "unit": "Tminplus/s", "frac": ach / peak_alu if peak_alu else None,
-                "traffic": ncu_traffic("k_fw_tiles", args.config),
+                "traffic": ncu_traffic("k_fw_tiles<Frag32>", args.config),
                 "avg_launch_ms": p3_ms / n_p3, "minplus_per_launch": prof["fw_phase3_minplus"] / n_p3,
                 "peak_basis": f"{SM_COUNT} SMs x {ALU_LANES_PER_SM} VIADDMNMX/clk/SM x {sm_max:.0f} MHz "
                               "(sm_max_mhz of MEASURED_PEAKS.json; issue rate from microbench/minplus_peak.cu)"}
@@ -349,8 +349,8 @@ def run_ours(args, rank, world, local_rank):
         n16 = max(int(prof["fw_phase3_launches"]), 1)
         ach = prof["fw_phase3_16_minplus"] / (p16 / 1e3) / 1e12
         peak_alu = SM_COUNT * lanes * sm_max * 1e6 / 1e12
-        roofline.update({"kernel": "k_fw_tiles16 (FW phase 3, packed u16x2)", "achieved": ach, "peak": peak_alu,
-                         "frac": ach / peak_alu, "traffic": ncu_traffic("k_fw_tiles16", args.config),
+        roofline.update({"kernel": "k_fw_tiles<Frag16> (FW phase 3, packed u16x2)", "achieved": ach, "peak": peak_alu,
+                         "frac": ach / peak_alu, "traffic": ncu_traffic("k_fw_tiles<Frag16>", args.config),
                          "avg_launch_ms": p16 / n16, "minplus_per_launch": prof["fw_phase3_16_minplus"] / n16,
                          "peak_basis": f"{SM_COUNT} SMs x {lanes} min-plus/clk/SM (64 VIADDMNMX.U16x2, two lanes "
                                        f"each) x {sm_max:.0f} MHz (sm_max_mhz of MEASURED_PEAKS.json; issue rate "
@@ -360,8 +360,8 @@ def run_ours(args, rank, world, local_rank):
     hbm = float(peaks.get("hbm_gbs", 6555.2))
     ex_ms = prof["expand_ms"]
     ex_ach = prof["expand_bytes"] / (ex_ms / 1e3) / 1e9 if ex_ms > 0 else 0.0
-    roofline_expand = {"bound": "hbm", "kernel": "k_expand", "achieved": ex_ach, "peak": hbm, "unit": "GB/s",
-                       "frac": ex_ach / hbm, "traffic": ncu_traffic("k_expand", args.config),
+    roofline_expand = {"bound": "hbm", "kernel": "k_expand_pairs", "achieved": ex_ach, "peak": hbm, "unit": "GB/s",
+                       "frac": ex_ach / hbm, "traffic": ncu_traffic("k_expand_pairs", args.config),
                        "avg_launch_ms": ex_ms / max(prof["expand_launches"], 1),
                        "bytes_per_launch": prof["expand_bytes"] / max(prof["expand_launches"], 1)}
     K = args.steps

@@ -16,7 +16,7 @@
 //                    e = uv whose tree paths meet only at z (LCA(u,v) = z), the cycle C_ze of weight
 //                    d_z(u) + W(uv) + d_z(v); sorted by weight once.
 //   phases           f = m - n + k phases; phase i: the labels l_z(u) = <path_z(u), S_i> of Algorithm 3
-//                    (one CTA per tree, level by level from the root); the first candidate in
+//                    (one warp per tree, level by level from the root); the first candidate in
 //                    weight order with l_z(u) xor l_z(v) xor S_i(e) = 1 (persistent CTAs over
 //                    batches with an early exit, no host round trip); C_i's incidence vector on E'
 //                    (walk of its two tree paths); the independence test S_j ^= S_i for every later
@@ -252,32 +252,33 @@ __global__ void k_witness_init(int32_t f, int32_t Wd, uint32_t *S) {
 }
 
 // ---- phase i, 1: labels l_z(u) = l_z(parent) xor S_i(parent edge) (0 for tree edges of T, which have
-// no coordinate), Algorithm 3; one CTA per tree, level by level; bit-packed into Lbits[z]
-__global__ void __launch_bounds__(NT) k_labels(int32_t N, int32_t L, const int32_t *__restrict__ order,
-                                               const int32_t *__restrict__ start, const int32_t *__restrict__ PE,
-                                               const int32_t *__restrict__ eu, const int32_t *__restrict__ ev,
-                                               const int32_t *__restrict__ coord, const uint32_t *__restrict__ Si,
-                                               uint32_t *__restrict__ Lbits, int32_t Wn) {
-  extern __shared__ uint8_t lab[];   // [N]
-  const int32_t z = blockIdx.x;
+// no coordinate), Algorithm 3; one WARP per tree, level by level (a warp barrier per level), the labels
+// as bits in shared memory (N bits per tree), then copied to Lbits[z]
+constexpr int LW = 8;   // trees (warps) per CTA
+__global__ void __launch_bounds__(LW * 32) k_labels(int32_t N, int32_t L, const int32_t *__restrict__ order,
+                                                    const int32_t *__restrict__ start, const int32_t *__restrict__ PE,
+                                                    const int32_t *__restrict__ eu, const int32_t *__restrict__ ev,
+                                                    const int32_t *__restrict__ coord, const uint32_t *__restrict__ Si,
+                                                    uint32_t *__restrict__ Lbits, int32_t Wn) {
+  extern __shared__ uint32_t lbits[];   // [LW][Wn]
+  const int lane = threadIdx.x & 31, wi = threadIdx.x >> 5;
+  const int32_t z = blockIdx.x * LW + wi;
+  if (z >= N) return;
+  uint32_t *lab = lbits + wi * Wn;
   const int32_t *ord = order + (int64_t)z * N, *st = start + (int64_t)z * (L + 1), *P = PE + (int64_t)z * N;
-  for (int32_t u = threadIdx.x; u < N; u += blockDim.x) lab[u] = 0;
-  __syncthreads();
+  for (int32_t w = lane; w < Wn; w += 32) lab[w] = 0;
+  __syncwarp();
   for (int32_t d = 1; d < L; ++d) {
     const int32_t b = st[d], e = st[d + 1];
     if (b == e) break;
-    for (int32_t idx = b + threadIdx.x; idx < e; idx += blockDim.x) {
+    for (int32_t idx = b + lane; idx < e; idx += 32) {
       const int32_t u = ord[idx], pe = P[u];
       const int32_t p = other_end(eu, ev, pe, u), c = coord[pe];
-      lab[u] = lab[p] ^ (uint8_t)(c >= 0 ? bit(Si, c) : 0u);
+      if (bit(lab, p) ^ (c >= 0 ? bit(Si, c) : 0u)) atomicOr(&lab[u >> 5], 1u << (u & 31));
     }
-    __syncthreads();
+    __syncwarp();
   }
-  for (int32_t w = threadIdx.x; w < Wn; w += blockDim.x) {
-    uint32_t x = 0;
-    for (int32_t j = 0; j < 32 && w * 32 + j < N; ++j) x |= (uint32_t)lab[w * 32 + j] << j;
-    Lbits[(int64_t)z * Wn + w] = x;
-  }
+  for (int32_t w = lane; w < Wn; w += 32) Lbits[(int64_t)z * Wn + w] = lab[w];
 }
 
 struct PhaseState {
@@ -629,12 +630,14 @@ ear_status_t mcb_build(ear_mcb_s *m, int32_t n, int64_t mm, const int32_t *src, 
   EAR_TRY(sc.get(&ps, 1));
   EAR_LAUNCH(k_witness_init, grid_for((int64_t)f * Wd), NT, 0, st)(f, Wd, S);
   EAR_LAUNCH(k_ps_init, 1, 1, 0, st)(ps);
-  EAR_CUDA_TRY(smem_attr((const void *)k_labels, N));
+  const int lsmem = LW * Wn * 4;
+  EAR_CUDA_TRY(smem_attr((const void *)k_labels, lsmem));
   const int scan_grid = num_sms() * 4;
   const int upd_grid = (int)std::max<int64_t>(1, std::min<int64_t>(ceil_div((int64_t)f * 32, NT), 148 * 8));
   for (int32_t i = 0; i < f; ++i) {
     const uint32_t *Si = S + (int64_t)i * Wd;
-    EAR_LAUNCH(k_labels, N, NT, N, st)(N, L, order, lstart, m->PE, m->eu, m->ev, coord, Si, Lbits, Wn);
+    EAR_LAUNCH(k_labels, (int)ceil_div(N, LW), LW * 32, lsmem, st)(N, L, order, lstart, m->PE, m->eu, m->ev, coord, Si,
+                                                                  Lbits, Wn);
     EAR_LAUNCH(k_scan, scan_grid, NT, 0, st)(m->ncand, dv.Current(), m->eu, m->ev, coord, Si, Lbits, Wn, ps);
     EAR_LAUNCH(k_cycle, 1, 128, 0, st)(i, dk.Current(), dv.Current(), m->eu, m->ev, m->PE, coord, N, C, Wd, ps,
                                        m->cyc_z, m->cyc_e, m->cyc_w);
