@@ -391,8 +391,9 @@ __global__ void __launch_bounds__(XP_NT, 1)
     int32_t pj = X.istart[v], rj = pj < pe ? X.pstart[pj] : 0;
     bool loaded_v = false;
     for (;;) {
-      if (tid == 0) {   // the next sweep: up to gcap partner rows and XP_RMAX chain rows in range
-        int ns = 0, nrow = 0;
+      if (tid < 32) {   // warp 0 builds the next sweep: up to gcap partner rows, XP_RMAX chain rows in range
+        const int lane = tid;
+        int ns = 0, nrow = 0;   // warp-uniform
         while (pj < pe && nrow < XP_RMAX) {
           const int32_t x = X.px[pj];
           int slot = 0;
@@ -402,17 +403,37 @@ __global__ void __launch_bounds__(XP_NT, 1)
               if (slot_x[k] == x) slot = k + 1;
             if (slot < 0) {
               if (ns == gcap) break;
-              slot_x[ns++] = x;
-              slot = ns;
+              if (lane == 0) slot_x[ns] = x;
+              __syncwarp();   // the other lanes read slot_x in the next partner's lookup
+              slot = ++ns;
             }
           }
           const int32_t r1 = X.pstart[pj + 1];
-          while (rj < r1 && nrow < XP_RMAX) {
-            const int32_t s = X.rows[rj++];
-            if (s >= rb && s < re) {
-              const VDesc d = desc[s];
-              const bool left = d.p == v;   // c_sv: along-chain distance from s to v
-              meta[nrow++] = make_int4(left ? d.cp : d.cq, left ? d.cq : d.cp, slot, s - rb);
+          while (rj < r1 && nrow < XP_RMAX) {   // 32 rows of the pair at a time
+            const int32_t idx = rj + lane;
+            bool in = false;
+            int4 mm = make_int4(0, 0, 0, 0);
+            if (idx < r1) {
+              const int32_t srow = X.rows[idx];
+              in = srow >= rb && srow < re;
+              if (in) {
+                const VDesc d = desc[srow];
+                const bool left = d.p == v;   // c_sv: along-chain distance from s to v
+                mm = make_int4(left ? d.cp : d.cq, left ? d.cq : d.cp, slot, srow - rb);
+              }
+            }
+            const unsigned bal = __ballot_sync(0xFFFFFFFFu, in);
+            const int cap = XP_RMAX - nrow, cnt = __popc(bal);
+            const int pos = __popc(bal & ((1u << lane) - 1u));
+            if (in && pos < cap) meta[nrow + pos] = mm;
+            if (cnt <= cap) {
+              rj = min(r1, rj + 32);
+              nrow += cnt;
+            } else {   // full: resume right after the cap-th row in range
+              unsigned b = bal;
+              for (int q = 0; q < cap - 1; ++q) b &= b - 1u;
+              rj += __ffs(b);
+              nrow = XP_RMAX;
             }
           }
           if (rj >= r1) {
@@ -420,7 +441,8 @@ __global__ void __launch_bounds__(XP_NT, 1)
             if (pj < pe) rj = X.pstart[pj];
           }
         }
-        s_nrow = nrow; s_ns = ns; s_pj = pj; s_rj = rj;
+        __syncwarp();
+        if (lane == 0) { s_nrow = nrow; s_ns = ns; s_pj = pj; s_rj = rj; }
       }
       __syncthreads();
       const int nrow = s_nrow, ns = s_ns;

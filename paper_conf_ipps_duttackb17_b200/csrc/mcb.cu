@@ -87,6 +87,20 @@ __global__ void k_direct_edges(int64_t A, const int32_t *ru, const int32_t *rv, 
       eu[e] = ru[a]; ev[e] = rv[a]; ew[e] = rw[a]; ech[e] = -1;
     }
 }
+__global__ void k_edge_keys(int32_t k, const int32_t *eu, const int32_t *ev, const int32_t *ew, uint64_t *key,
+                            int32_t *w) {
+  for (int32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < k; i += gridDim.x * blockDim.x) {
+    key[i] = ((uint64_t)(uint32_t)eu[i] << 32) | (uint32_t)ev[i];
+    w[i] = ew[i];
+  }
+}
+__global__ void k_edge_unkey(int32_t k, const uint64_t *key, const int32_t *w, int32_t *eu, int32_t *ev, int32_t *ew) {
+  for (int32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < k; i += gridDim.x * blockDim.x) {
+    eu[i] = (int32_t)(key[i] >> 32);
+    ev[i] = (int32_t)(key[i] & 0xFFFFFFFFu);
+    ew[i] = w[i];
+  }
+}
 // CSR of G^r (both arc directions; a self-loop gives two arcs at its vertex, never tight)
 __global__ void k_deg(int64_t M, const int32_t *eu, const int32_t *ev, int32_t *deg) {
   for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < M; e += (int64_t)gridDim.x * blockDim.x) {
@@ -193,6 +207,20 @@ __global__ void k_level_scatter(int32_t N, int32_t L, const int32_t *depth, cons
     order[z * N + p] = (int32_t)(i % N);
   }
 }
+// the level order with what a label step needs per node: {u, parent, coordinate of the parent edge
+// (-1 for tree edges of T), 0} -- one 16-byte load per node in k_labels
+__global__ void k_order4(int32_t N, int32_t L, const int32_t *order, const int32_t *lstart, const int32_t *PE,
+                         const int32_t *eu, const int32_t *ev, const int32_t *coord, int4 *ord4) {
+  const int64_t NN = (int64_t)N * N;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < NN; i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t z = i / N;
+    const int32_t idx = (int32_t)(i % N);
+    if (idx < lstart[z * (L + 1) + 1] || idx >= lstart[z * (L + 1) + L]) continue;   // the root, unreachable
+    const int32_t u = order[i], pe = PE[z * N + u];
+    ord4[i] = make_int4(u, other_end(eu, ev, pe, u), coord[pe], 0);
+  }
+}
+
 // the fixed spanning forest T: the tree of each component's smallest vertex; E' coordinates
 __global__ void k_mark_tree(int32_t N, const int32_t *lab, const int32_t *PE, int32_t *intree, int32_t *roots) {
   for (int32_t u = blockIdx.x * blockDim.x + threadIdx.x; u < N; u += gridDim.x * blockDim.x) {
@@ -255,26 +283,24 @@ __global__ void k_witness_init(int32_t f, int32_t Wd, uint32_t *S) {
 // no coordinate), Algorithm 3; one WARP per tree, level by level (a warp barrier per level), the labels
 // as bits in shared memory (N bits per tree), then copied to Lbits[z]
 constexpr int LW = 8;   // trees (warps) per CTA
-__global__ void __launch_bounds__(LW * 32) k_labels(int32_t N, int32_t L, const int32_t *__restrict__ order,
-                                                    const int32_t *__restrict__ start, const int32_t *__restrict__ PE,
-                                                    const int32_t *__restrict__ eu, const int32_t *__restrict__ ev,
-                                                    const int32_t *__restrict__ coord, const uint32_t *__restrict__ Si,
+__global__ void __launch_bounds__(LW * 32) k_labels(int32_t N, int32_t L, const int4 *__restrict__ ord4,
+                                                    const int32_t *__restrict__ start, const uint32_t *__restrict__ Si,
                                                     uint32_t *__restrict__ Lbits, int32_t Wn) {
   extern __shared__ uint32_t lbits[];   // [LW][Wn]
   const int lane = threadIdx.x & 31, wi = threadIdx.x >> 5;
   const int32_t z = blockIdx.x * LW + wi;
   if (z >= N) return;
   uint32_t *lab = lbits + wi * Wn;
-  const int32_t *ord = order + (int64_t)z * N, *st = start + (int64_t)z * (L + 1), *P = PE + (int64_t)z * N;
+  const int4 *ord = ord4 + (int64_t)z * N;
+  const int32_t *st = start + (int64_t)z * (L + 1);
   for (int32_t w = lane; w < Wn; w += 32) lab[w] = 0;
   __syncwarp();
   for (int32_t d = 1; d < L; ++d) {
     const int32_t b = st[d], e = st[d + 1];
     if (b == e) break;
     for (int32_t idx = b + lane; idx < e; idx += 32) {
-      const int32_t u = ord[idx], pe = P[u];
-      const int32_t p = other_end(eu, ev, pe, u), c = coord[pe];
-      if (bit(lab, p) ^ (c >= 0 ? bit(Si, c) : 0u)) atomicOr(&lab[u >> 5], 1u << (u & 31));
+      const int4 r = ord[idx];   // {u, parent, coordinate of the parent edge or -1}
+      if (bit(lab, r.y) ^ (r.z >= 0 ? bit(Si, r.z) : 0u)) atomicOr(&lab[r.x >> 5], 1u << (r.x & 31));
     }
     __syncwarp();
   }
@@ -509,9 +535,29 @@ ear_status_t mcb_build(ear_mcb_s *m, int32_t n, int64_t mm, const int32_t *src, 
   if (p->n_chains > 0)
     EAR_LAUNCH(k_chain_edges, grid_for(p->n_chains), NT, 0, st)(p->n_chains, p->seg_start, p->seg_vert, p->desc, m->eu,
                                                                  m->ev, m->ew, m->ech);
-  if (ndirect > 0)
+  if (ndirect > 0) {
     EAR_LAUNCH(k_direct_edges, grid_for(p->n_redges), NT, 0, st)(p->n_redges, p->re_u, p->re_v, p->re_w, dflag, dpos,
                                                                   p->n_chains, m->eu, m->ev, m->ew, m->ech);
+    // Phase I emits the reduced arcs in atomic order: number the direct edges by (u, v) instead, so that
+    // edge ids -- hence the perturbation and every tie-break -- are the same on every run
+    uint64_t *k0 = nullptr, *k1 = nullptr;
+    int32_t *w0 = nullptr, *w1 = nullptr;
+    EAR_TRY(sc.get(&k0, ndirect));
+    EAR_TRY(sc.get(&k1, ndirect));
+    EAR_TRY(sc.get(&w0, ndirect));
+    EAR_TRY(sc.get(&w1, ndirect));
+    const int32_t c0 = p->n_chains;
+    EAR_LAUNCH(k_edge_keys, grid_for(ndirect), NT, 0, st)(ndirect, m->eu + c0, m->ev + c0, m->ew + c0, k0, w0);
+    cub::DoubleBuffer<uint64_t> dk(k0, k1);
+    cub::DoubleBuffer<int32_t> dw(w0, w1);
+    size_t tb = 0;
+    EAR_CUDA_TRY(cub::DeviceRadixSort::SortPairs(nullptr, tb, dk, dw, ndirect, 0, 64, st));
+    char *tmp = nullptr;
+    EAR_TRY(sc.get(&tmp, (int64_t)tb));
+    EAR_CUDA_TRY(cub::DeviceRadixSort::SortPairs(tmp, tb, dk, dw, ndirect, 0, 64, st));
+    EAR_LAUNCH(k_edge_unkey, grid_for(ndirect), NT, 0, st)(ndirect, dk.Current(), dw.Current(), m->eu + c0, m->ev + c0,
+                                                           m->ew + c0);
+  }
   EAR_TRY(alloc_keep(&m->tid2v, N, st));
   EAR_LAUNCH(k_tid2v, grid_for(n), NT, 0, st)(n, p->tid, m->tid2v);
   // CSR
@@ -583,6 +629,9 @@ ear_status_t mcb_build(ear_mcb_s *m, int32_t n, int64_t mm, const int32_t *src, 
     EAR_TRY(read1(&lf, nflag + M - 1, st));
     f = lp + lf;
   }
+  int4 *ord4 = nullptr;
+  EAR_TRY(sc.get(&ord4, NN));
+  EAR_LAUNCH(k_order4, grid_for(NN), NT, 0, st)(N, L, order, lstart, m->PE, m->eu, m->ev, coord, ord4);
   EAR_TRY(read1(&m->k, roots, st));
   m->f = f;
   if ((int64_t)f != M - N + m->k) {
@@ -611,13 +660,26 @@ ear_status_t mcb_build(ear_mcb_s *m, int32_t n, int64_t mm, const int32_t *src, 
   EAR_TRY(sc.get(&v1, m->ncand));
   EAR_CUDA_TRY(dev_memset(cnt, 0, sizeof(unsigned long long), st));
   EAR_LAUNCH(k_candidates, grid_for(NM), NT, 0, st)(N, M, Np, D, m->eu, m->ev, m->ew, m->PE, BR, H, cnt, k0, v0);
+  // k_candidates emits in atomic order and equal keys (one cycle found from several roots) are common:
+  // order by (z, e) first, then the stable sort by key leaves every tie in that order -- the same basis,
+  // with the same root per cycle, on every run
   cub::DoubleBuffer<uint64_t> dk(k0, k1);
   cub::DoubleBuffer<int64_t> dv(v0, v1);
   {
-    size_t tb = 0;
+    uint64_t *u0 = reinterpret_cast<uint64_t *>(v0), *u1 = reinterpret_cast<uint64_t *>(v1);
+    int64_t *s0 = reinterpret_cast<int64_t *>(k0), *s1 = reinterpret_cast<int64_t *>(k1);
+    cub::DoubleBuffer<uint64_t> dz(u0, u1);   // (z, e) as the key, the candidate key as the value
+    cub::DoubleBuffer<int64_t> dy(s0, s1);
+    size_t tb = 0, tb2 = 0;
     EAR_CUDA_TRY(cub::DeviceRadixSort::SortPairs(nullptr, tb, dk, dv, m->ncand, 0, 64, st));
+    EAR_CUDA_TRY(cub::DeviceRadixSort::SortPairs(nullptr, tb2, dz, dy, m->ncand, 0, 64, st));
     char *tmp = nullptr;
-    EAR_TRY(sc.get(&tmp, (int64_t)tb));
+    EAR_TRY(sc.get(&tmp, (int64_t)std::max(tb, tb2)));
+    EAR_CUDA_TRY(cub::DeviceRadixSort::SortPairs(tmp, tb2, dz, dy, m->ncand, 0, 64, st));
+    dk = cub::DoubleBuffer<uint64_t>(reinterpret_cast<uint64_t *>(dy.Current()),
+                                     reinterpret_cast<uint64_t *>(dy.Alternate()));
+    dv = cub::DoubleBuffer<int64_t>(reinterpret_cast<int64_t *>(dz.Current()),
+                                    reinterpret_cast<int64_t *>(dz.Alternate()));
     EAR_CUDA_TRY(cub::DeviceRadixSort::SortPairs(tmp, tb, dk, dv, m->ncand, 0, 64, st));
   }
   // ---- phases
@@ -636,8 +698,7 @@ ear_status_t mcb_build(ear_mcb_s *m, int32_t n, int64_t mm, const int32_t *src, 
   const int upd_grid = (int)std::max<int64_t>(1, std::min<int64_t>(ceil_div((int64_t)f * 32, NT), 148 * 8));
   for (int32_t i = 0; i < f; ++i) {
     const uint32_t *Si = S + (int64_t)i * Wd;
-    EAR_LAUNCH(k_labels, (int)ceil_div(N, LW), LW * 32, lsmem, st)(N, L, order, lstart, m->PE, m->eu, m->ev, coord, Si,
-                                                                  Lbits, Wn);
+    EAR_LAUNCH(k_labels, (int)ceil_div(N, LW), LW * 32, lsmem, st)(N, L, ord4, lstart, Si, Lbits, Wn);
     EAR_LAUNCH(k_scan, scan_grid, NT, 0, st)(m->ncand, dv.Current(), m->eu, m->ev, coord, Si, Lbits, Wn, ps);
     EAR_LAUNCH(k_cycle, 1, 128, 0, st)(i, dk.Current(), dv.Current(), m->eu, m->ev, m->PE, coord, N, C, Wd, ps,
                                        m->cyc_z, m->cyc_e, m->cyc_w);

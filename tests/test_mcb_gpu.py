@@ -148,3 +148,17 @@ def test_mcb_degenerate(ea, case):
         g = gg.torus(6, 7, 10, seed=9)
         n, src, dst, w = g.n, g.src, g.dst, np.ones_like(g.w)
     check_mcb(ea, n, src, dst, w)
+
+
+def test_mcb_deterministic(ea):
+    """Two builds of the same graph choose the same trees, candidates and basis (the perturbation of
+    reading M3 is a fixed hash; every tie is broken by the edge id)."""
+    g = gg.config("cfg1")
+    runs = []
+    for _ in range(2):
+        r = ea.mcb(g.n, dev(g.src), dev(g.dst), dev(g.w))
+        runs.append((r.info(), r.weights().cpu().numpy(), [r.cycle(i).cpu().numpy().tolist() for i in (0, 7, 500)]))
+        r.destroy()
+    assert runs[0][0] == runs[1][0]
+    assert np.array_equal(runs[0][1], runs[1][1])
+    assert runs[0][2] == runs[1][2]

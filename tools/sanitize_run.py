@@ -1,8 +1,10 @@
 """Small end-to-end runs for compute-sanitizer (memcheck / racecheck / synccheck): every kernel of the
-library on graphs small enough for the instrumented run -- packed and int32 FW (single + emulated
-sharding with the owner-side phase 2 and lookahead), blocks with a re-reduced piece, SSSP, expansion
-(aligned and scalar store paths), query mode, Phase I with pure cycles, the host-buffer entry points
-(two async jobs in flight, pinned and pageable inputs)."""
+library on graphs small enough for the instrumented run -- packed and int32 FW (single, emulated
+sharding with the owner-side phase 2 and lookahead, and a one-rank communicator: window pushes, flags,
+the pull gather), blocks with a re-reduced piece (u16 compose route), SSSP, expansion (pair-major on
+aligned rows, row-group on unaligned rows), query mode, Phase I with pure cycles, the MCB (trees,
+candidates, phases, cycle expansion), the host-buffer entry points (two async jobs in flight, pinned
+and pageable inputs)."""
 import sys
 
 import numpy as np
@@ -27,6 +29,17 @@ for g in [gg.corner_cases(5, n_target=300), gg.torus(12, 12, 150, seed=1), gg.cy
     ea.expand_ears(plan, D, 0, g.n, out=big[:, 1:1 + g.n])
     s = dev(np.arange(g.n)); t = dev(np.arange(g.n)[::-1].copy())
     ea.query_pairs(plan, D, s, t)
+    aligned = torch.zeros((g.n, (g.n + 3) // 4 * 4), dtype=torch.int32, device="cuda")
+    ea.expand_ears(plan, D, 0, g.n, out=aligned[:, :g.n])          # pair-major kernel (aligned rows)
+    mc = ea.mcb(g.n, dev(g.src), dev(g.dst), dev(g.w))
+    for i in range(min(3, mc.info()["dim"])):
+        mc.cycle(i)
+    mc.destroy()
+comm = ea.Comm.single()   # the sharded schedule through its window: pushes, flags, pull gather
+for g in [gg.corner_cases(5, n_target=300), gg.torus(12, 12, 150, seed=1)]:
+    for flags in (0, ea.FLAG_FW32, ea.FLAG_BCC):
+        ea.apsp_full(g.n, dev(g.src), dev(g.dst), dev(g.w), flags=flags, comm=comm)
+comm.destroy()
 # host-buffer entry points, two async jobs in flight (mapped-pinned readbacks, kernel memsets)
 g = gg.corner_cases(5, n_target=300)
 hs, hd, hw = (torch.as_tensor(np.ascontiguousarray(a, dtype=np.int32)).pin_memory() for a in (g.src, g.dst, g.w))
