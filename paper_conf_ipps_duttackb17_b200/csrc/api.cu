@@ -329,6 +329,17 @@ static ear_status_t solve_rows(ear_plan_s *p, int32_t row_begin, int32_t row_end
       k.D16 = nullptr;
     }
   }
+  if (!comm && (p->flags & EAR_FLAG_SSSP) && u16_ok && xp_applicable(p, st)) {
+    // per-source SSSP straight into u16 rows: no int32 D, no narrowing pass
+    k.ld16 = xp_row_stride(p);
+    EAR_CUDA_TRY(cudaMallocAsync((void **)&k.D16, sizeof(uint16_t) * (size_t)p->n_reduced * k.ld16, st));
+    bool applied = false;
+    s = sssp_rows16(p, k.D16, k.ld16, &applied, st);
+    if (s != EAR_OK || !applied) {
+      cudaFreeAsync(k.D16, st);
+      k.D16 = nullptr;
+    }
+  }
   if (s == EAR_OK && !k.D16) {
     if (!comm) {
       EAR_CUDA_TRY(cudaMallocAsync((void **)&k.D, sizeof(int32_t) * (size_t)Np * Np, st));

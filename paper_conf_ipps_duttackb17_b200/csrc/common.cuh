@@ -80,6 +80,9 @@ struct ear_plan_s {
   int32_t *r_rowptr = nullptr, *r_col = nullptr, *r_w = nullptr;
   void *r_arcs = nullptr;       // packed (col, w) int2 arcs: ELL rows of r_ell_k per vertex, or CSR order
   int32_t r_ell_k = -1;
+  uint32_t *r_ell16 = nullptr;  // u16 route: ELL rows of r_k16 packed arcs (target | min(w, 0xFFFF) << 16)
+  int32_t r_k16 = -1;           // 0: the u16 route does not apply (N_r >= 0xFFFF or a degree > 16)
+  uint32_t r_delta = 0;         // near-far step of the u16 SSSP (16 x the mean arc weight)
   int32_t n_rarcs = 0;
   ear_bcc_s *bcc = nullptr;     // built on first use (EAR_FLAG_BCC, ear_bcc_info)
   int32_t *cc = nullptr;        // [cc_np] connected-component labels of G^r (16-bit FW range check)
@@ -171,6 +174,9 @@ ear_status_t shard_rows_device(int32_t nt, int32_t P, int32_t rank, int32_t **d_
 // holds global rows d_tile_rows[b]*128 ..), written consecutively into D
 ear_status_t sssp_rows(ear_plan_s *plan, int32_t *D, int64_t ldd, int32_t Np, int32_t row0, int32_t rows,
                        const int32_t *d_tile_rows, cudaStream_t stream);
+// every row of D (reduced vertex order, 0xFFFF = INF, stride ld16 >= round_up(N_r, 8)) by the u16 SSSP;
+// *applied = false when the route does not apply or a finite distance >= 0xFFFF exists (D16 unusable)
+ear_status_t sssp_rows16(ear_plan_s *plan, uint16_t *D16, int64_t ld16, bool *applied, cudaStream_t stream);
 // bcc.cu -- Phase II by biconnected pieces (paper sec. 2.2)
 ear_status_t bcc_prepare(ear_plan_s *plan, int32_t P, cudaStream_t stream);
 // D16 / ld16 / flag16 (optional): also (or, with D == NULL, only) the rows as u16 for the pair-major

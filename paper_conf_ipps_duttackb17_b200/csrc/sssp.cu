@@ -385,6 +385,301 @@ __global__ void __launch_bounds__(NTS) k_sssp_list(const int2 *__restrict__ ell,
   }
 }
 
+// ---- the u16 route: distances below 0xFFFF, N_r < 0xFFFF (cfg1-cfg4 of the paper's workloads).
+// One CTA per source at a time (persistent, sources from a counter), the distance row in shared memory
+// as DistT: u16 (half the bytes: more sources per SM; 16-bit CAS relaxations) or u32 (one ATOMS.MIN per
+// relaxation).  One barrier per round: round r expands the list of round r and appends improved
+// vertices to round r+1's, deduped by the bitmap M[(r+1)%2] (round r+1 zeroes it while it expands: sets
+// and clears of a bitmap are a barrier apart, so no fence is needed -- a vertex improved before its own
+// expansion in the same round is expanded once more next round, harmlessly).
+// Work is counted in warp instructions (ncu: the kernel is issue-bound), so: the list is cut into
+// 32-entry tasks and only warps holding a task run; a warp walks its vertices' ELL slots only while
+// some lane still has a real arc (padding sits at the row end); the lists are split into one segment
+// per warp and appended WARP-SYNCHRONOUSLY -- after each slot the warp ballots its new vertices and
+// writes them at a register-held offset (no shared counter: same-address atomics serialise).  A
+// segment that overflows makes the next round scan its bitmap instead.  Arcs are ELL rows of K packed
+// u32 (target | weight << 16; padding target 0xFFFF).  A candidate >= 0xFFFF for a still-unreached
+// vertex marks the source, and a marked source whose row keeps an unreached vertex raises *sat: the
+// caller then falls back to int32 (every shortest path's prefixes are below the final distance, so a
+// row without unreached vertices is exact).
+template <typename DistT>
+__device__ __forceinline__ bool sssp_lower(DistT *d, uint32_t nd, uint32_t cur) {
+  if constexpr (sizeof(DistT) == 4) {
+    return nd < atomicMin(reinterpret_cast<unsigned int *>(d), nd);
+  } else {
+    for (;;) {
+      const uint16_t old = atomicCAS(reinterpret_cast<unsigned short *>(d), (uint16_t)cur, (uint16_t)nd);
+      if (old == (uint16_t)cur) return true;
+      cur = old;
+      if (nd >= cur) return false;
+    }
+  }
+}
+
+template <int NTS, int K, int J, typename DistT, typename OutT>
+__global__ void __launch_bounds__(NTS) k_sssp16(const uint4 *__restrict__ ell, int32_t nr, int32_t L, OutT *out,
+                                               int64_t ldo, int32_t src0, int32_t nsrc, const int32_t *trows, int cap,
+                                               uint32_t delta, int32_t *counter, int32_t *sat,
+                                               unsigned long long *stats) {
+  constexpr int NW = NTS / 32;
+  constexpr uint32_t DINF = sizeof(DistT) == 2 ? 0xFFFFu : 0xFFFFFFFFu;
+  extern __shared__ __align__(16) uint32_t smw[];
+  const int W = (L + 31) >> 5;
+  const int S = cap / NW;                                                    // segment length
+  DistT *dist = reinterpret_cast<DistT *>(smw);                              // [L], L % 8 == 0
+  uint32_t *Mb = reinterpret_cast<uint32_t *>(dist + L);                     // [2][W]
+  uint32_t *F = Mb + 2 * W;                                                  // [W] the far pile
+  uint16_t *Lb = reinterpret_cast<uint16_t *>(F + W);                        // [2][NW][S]
+  __shared__ int scnt[3][NW], ovf[3], s_item, s_sat;
+  __shared__ uint32_t s_min[NW];
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const uint32_t lt = (1u << lane) - 1u;
+  const int wpt = (W + NTS - 1) / NTS, w0 = tid * wpt, w1 = min(W, w0 + wpt);   // owned bitmap words
+  unsigned long long my_rounds = 0, my_relax = 0;
+  for (;;) {
+    if (tid == 0) s_item = atomicAdd(counter, 1);
+    __syncthreads();
+    const int32_t li = s_item;
+    if (li >= nsrc) break;
+    const int32_t src = trows ? trows[li >> 7] * TILE + (li & (TILE - 1)) : src0 + li;
+    for (int i = tid; i < L * (int)sizeof(DistT) / 16; i += NTS)
+      reinterpret_cast<uint4 *>(dist)[i] = make_uint4(~0u, ~0u, ~0u, ~0u);
+    for (int w = tid; w < 3 * W; w += NTS) Mb[w] = 0u;   // both list bitmaps and F
+    if (tid < 3 * NW) (&scnt[0][0])[tid] = 0;
+    if (tid < 3) ovf[tid] = 0;
+    if (tid == 0) s_sat = 0;
+    __syncthreads();
+    if (tid == 0) {
+      dist[src] = 0;   // a padding source (src >= nr) has no arcs: its row is INF but the diagonal
+      Lb[0] = (uint16_t)src;
+      Mb[src >> 5] = 1u << (src & 31);
+      scnt[0][0] = 1;
+    }
+    __syncthreads();
+    if (src < nr) {
+      uint32_t thr = delta;   // near-far: only vertices below thr are expanded (uniform)
+      for (int r = 0;; ++r) {
+        const uint16_t *Lc = Lb + (r & 1) * (NW * S);
+        uint16_t *Ln = Lb + ((r + 1) & 1) * (NW * S) + warp * S;   // this warp's segment
+        uint32_t *Mc = Mb + (r & 1) * W, *Mn = Mb + ((r + 1) & 1) * W;
+        const bool scan = ovf[r % 3] != 0;
+        int *ncnt = &scnt[(r + 1) % 3][warp];
+        int *novf = &ovf[(r + 1) % 3];
+        if (tid < NW) scnt[(r + 2) % 3][tid] = 0;
+        if (tid == 0) ovf[(r + 2) % 3] = 0;
+        // relax arc a from a vertex at distance dv; true when u is new on round r+1's list
+        auto relax = [&](uint32_t dv, uint32_t a) -> bool {
+          const uint32_t u = a & 0xFFFFu;
+          if (u == 0xFFFFu) return false;
+          const uint32_t nd = dv + (a >> 16);
+          const uint32_t cur = dist[u];
+          if (nd >= 0xFFFFu) {   // not representable: harmless unless u stays unreached
+            if (cur == DINF) s_sat = 1;
+            return false;
+          }
+          if (nd >= cur || !sssp_lower(dist + u, nd, cur)) return false;
+          if (stats) ++my_relax;
+          const uint32_t bit = 1u << (u & 31);
+          if (nd >= thr) {   // far: waits for the threshold
+            atomicOr(&F[u >> 5], bit);
+            return false;
+          }
+          return !(atomicOr(&Mn[u >> 5], bit) & bit);
+        };
+        if (!scan) {
+          int pre[NW + 1];
+          pre[0] = 0;
+#pragma unroll
+          for (int w = 0; w < NW; ++w) pre[w + 1] = pre[w] + min(scnt[r % 3][w], S);
+          const int n = pre[NW], ntask = (n + 31) >> 5;
+          for (int w = w0; w < w1; ++w) Mc[w] = 0u;   // nobody sets Mc this round
+          int wc = 0;                                 // warp-uniform append offset
+          for (int t0 = warp; t0 < ntask; t0 += J * NW) {   // warp-uniform: the ballots see all lanes
+            int vv[J];
+            uint4 e[J][K / 4];
+#pragma unroll
+            for (int j = 0; j < J; ++j) {
+              const int i = (t0 + j * NW) * 32 + lane;
+              vv[j] = -1;
+              if (i < n) {
+                int sg = 0;
+#pragma unroll
+                for (int w = 1; w < NW; ++w) sg += i >= pre[w];
+                vv[j] = Lc[sg * S + i - pre[sg]];
+              }
+              const uint4 *row = ell + (int64_t)max(vv[j], 0) * (K / 4);
+#pragma unroll
+              for (int k = 0; k < K / 4; ++k) e[j][k] = vv[j] >= 0 ? __ldg(row + k) : make_uint4(~0u, ~0u, ~0u, ~0u);
+            }
+#pragma unroll
+            for (int j = 0; j < J; ++j) {
+              if (t0 + j * NW >= ntask) break;
+              const uint32_t dv = vv[j] >= 0 ? (uint32_t)dist[vv[j]] : 0u;
+#pragma unroll
+              for (int k = 0; k < K; ++k) {
+                const uint4 q = e[j][k / 4];
+                const uint32_t a = (k & 3) == 0 ? q.x : (k & 3) == 1 ? q.y : (k & 3) == 2 ? q.z : q.w;
+                if (!__any_sync(0xFFFFFFFFu, (a & 0xFFFFu) != 0xFFFFu)) break;
+                const bool push = relax(dv, a);
+                const unsigned bal = __ballot_sync(0xFFFFFFFFu, push);
+                if (push) {
+                  const int idx = wc + __popc(bal & lt);
+                  if (idx < S) Ln[idx] = (uint16_t)(a & 0xFFFFu);
+                }
+                wc += __popc(bal);
+              }
+            }
+          }
+          if (lane == 0) {
+            *ncnt = wc;
+            if (wc > S) *novf = 1;
+          }
+        } else {   // an overflowed segment: the bitmap holds every vertex listed for this round
+          for (int w = w0; w < w1; ++w) {
+            uint32_t m = Mc[w];
+            Mc[w] = 0u;
+            while (m) {
+              const int b = __ffs(m) - 1;
+              m &= m - 1;
+              const int v = (w << 5) + b;
+              uint4 e[K / 4];
+#pragma unroll
+              for (int k = 0; k < K / 4; ++k) e[k] = __ldg(ell + (int64_t)v * (K / 4) + k);
+              const uint32_t dv = dist[v];
+#pragma unroll
+              for (int k = 0; k < K; ++k) {
+                const uint4 q = e[k / 4];
+                const uint32_t a = (k & 3) == 0 ? q.x : (k & 3) == 1 ? q.y : (k & 3) == 2 ? q.z : q.w;
+                if (relax(dv, a)) {
+                  const int idx = atomicAdd(ncnt, 1);
+                  if (idx < S) Ln[idx] = (uint16_t)(a & 0xFFFFu); else *novf = 1;
+                }
+              }
+            }
+          }
+        }
+        __syncthreads();
+        ++my_rounds;
+        int more = ovf[(r + 1) % 3];
+#pragma unroll
+        for (int w = 0; w < NW; ++w) more |= scnt[(r + 1) % 3][w];
+        if (more) continue;
+        // the near pile is empty: raise the threshold to (smallest live far distance) + delta and list
+        // the far vertices below it for round r+1.  A far entry already below the old threshold is stale
+        // (a later improvement put it on a near list): it is dropped.
+        uint32_t mn = 0xFFFFFFFFu;
+        for (int w = w0; w < w1; ++w) {
+          uint32_t m = F[w];
+          while (m) {
+            const int b = __ffs(m) - 1;
+            m &= m - 1;
+            const uint32_t d = dist[(w << 5) + b];
+            if (d >= thr) mn = min(mn, d);
+          }
+        }
+#pragma unroll
+        for (int o = 16; o; o >>= 1) mn = min(mn, __shfl_xor_sync(0xFFFFFFFFu, mn, o));
+        if (lane == 0) s_min[warp] = mn;
+        __syncthreads();
+        mn = 0xFFFFFFFFu;
+#pragma unroll
+        for (int w = 0; w < NW; ++w) mn = min(mn, s_min[w]);
+        if (mn == 0xFFFFFFFFu) break;   // no live far vertex: the row is final
+        const uint32_t told = thr;
+        thr = mn + delta;
+        {
+          uint32_t *Mn = Mb + ((r + 1) & 1) * W;   // round r+1's list bitmap (owned words: plain stores)
+          uint16_t *Ln = Lb + ((r + 1) & 1) * (NW * S) + warp * S;
+          int wc = 0;
+          for (int wb = warp * 32 * wpt; wb < W; wb += NTS * wpt) {   // warp-uniform over the owned words
+            for (int q = 0; q < wpt; ++q) {
+              const int w = wb + lane * wpt + q;
+              uint32_t m = w < W ? F[w] : 0u, take = 0u, stale = 0u;
+              for (uint32_t x = m; x; x &= x - 1) {
+                const int b = __ffs(x) - 1;
+                const uint32_t d = dist[(w << 5) + b];
+                if (d < told) stale |= 1u << b;
+                else if (d < thr) take |= 1u << b;
+              }
+              if (w < W) {
+                F[w] = m & ~(take | stale);
+                Mn[w] |= take;
+              }
+              while (__any_sync(0xFFFFFFFFu, take != 0u)) {
+                const bool has = take != 0u;
+                const int b = has ? __ffs(take) - 1 : 0;
+                take &= take - 1;
+                const unsigned bal = __ballot_sync(0xFFFFFFFFu, has);
+                if (has) {
+                  const int idx = wc + __popc(bal & lt);
+                  if (idx < S) Ln[idx] = (uint16_t)((w << 5) + b);
+                }
+                wc += __popc(bal);
+              }
+            }
+          }
+          if (lane == 0) {
+            scnt[(r + 1) % 3][warp] = wc;
+            if (wc > S) ovf[(r + 1) % 3] = 1;
+          }
+        }
+        __syncthreads();
+      }
+    }
+    if (s_sat) {   // uniform (read after the last round's barrier)
+      bool un = false;
+      for (int i = tid; i < nr; i += NTS) un |= dist[i] == DINF;
+      if (__syncthreads_or(un) && tid == 0) atomicOr(sat, 1);
+    }
+    OutT *row = out + (int64_t)li * ldo;
+    for (int i = tid; i < L / 8; i += NTS) {   // 8 entries per step
+      uint32_t x[8];
+      if constexpr (sizeof(DistT) == 2) {
+        const uint4 q = reinterpret_cast<const uint4 *>(dist)[i];
+        const uint32_t h[4] = {q.x, q.y, q.z, q.w};
+#pragma unroll
+        for (int k = 0; k < 4; ++k) { x[2 * k] = h[k] & 0xFFFFu; x[2 * k + 1] = h[k] >> 16; }
+      } else {
+        const uint4 q0 = reinterpret_cast<const uint4 *>(dist)[2 * i], q1 = reinterpret_cast<const uint4 *>(dist)[2 * i + 1];
+        x[0] = q0.x; x[1] = q0.y; x[2] = q0.z; x[3] = q0.w; x[4] = q1.x; x[5] = q1.y; x[6] = q1.z; x[7] = q1.w;
+      }
+      if constexpr (sizeof(OutT) == 2) {
+        uint32_t y[4];
+#pragma unroll
+        for (int k = 0; k < 4; ++k) y[k] = min(x[2 * k], 0xFFFFu) | (min(x[2 * k + 1], 0xFFFFu) << 16);
+        reinterpret_cast<uint4 *>(row)[i] = make_uint4(y[0], y[1], y[2], y[3]);
+      } else {
+        int32_t y[8];
+#pragma unroll
+        for (int k = 0; k < 8; ++k) y[k] = x[k] >= 0xFFFFu ? INF : (int32_t)x[k];
+        reinterpret_cast<int4 *>(row)[2 * i] = make_int4(y[0], y[1], y[2], y[3]);
+        reinterpret_cast<int4 *>(row)[2 * i + 1] = make_int4(y[4], y[5], y[6], y[7]);
+      }
+    }
+    __syncthreads();
+  }
+  if (stats) {
+    if (tid == 0) atomicAdd(&stats[0], my_rounds);
+    atomicAdd(&stats[1], my_relax);
+  }
+}
+
+__global__ void k_sum_w(const int32_t *w, int32_t A, unsigned long long *sum) {
+  unsigned long long t = 0;
+  for (int64_t a = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; a < A; a += (int64_t)gridDim.x * blockDim.x)
+    t += (unsigned long long)w[a];
+  atomicAdd(sum, t);
+}
+
+__global__ void k_build_ell16(const int32_t *rowptr, const int32_t *col, const int32_t *w, int32_t nr, int K,
+                              uint32_t *ell) {
+  for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < nr; v += (int64_t)gridDim.x * blockDim.x) {
+    const int a0 = rowptr[v], d = rowptr[v + 1] - a0;
+    for (int k = 0; k < K; ++k)
+      ell[v * K + k] = k < d ? ((uint32_t)col[a0 + k] | ((uint32_t)min(w[a0 + k], 0xFFFF) << 16)) : 0xFFFFFFFFu;
+  }
+}
+
 __global__ void k_build_ell(const int32_t *rowptr, const int32_t *col, const int32_t *w, int32_t nr, int K,
                             int2 *ell) {
   for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < nr; v += (int64_t)gridDim.x * blockDim.x) {
@@ -517,12 +812,173 @@ static ear_status_t sssp_list_launch(ear_plan_s *p, int32_t *D, int64_t ldd, int
   return EAR_OK;
 }
 
+// ---- u16 route (host side)
+static ear_status_t ell16_prepare(ear_plan_s *p, cudaStream_t st) {
+  if (p->r_k16 >= 0) return EAR_OK;
+  EAR_TRY(sssp_prepare(p, st));
+  const int32_t nr = p->n_reduced;
+  p->r_k16 = 0;
+  if (nr <= 0 || nr >= 0xFFFF) return EAR_OK;
+  int32_t *d_md = nullptr, md = 0;
+  unsigned long long wsum = 0;
+  EAR_CUDA_TRY(cudaMallocAsync((void **)&d_md, 16, st));
+  EAR_CUDA_TRY(dev_memset(d_md, 0, 16, st));
+  unsigned long long *d_sum = reinterpret_cast<unsigned long long *>(d_md + 2);
+  EAR_LAUNCH(k_max_deg, (int)std::min<int64_t>(ceil_div(nr, 256), 4096), 256, 0, st)(p->r_rowptr, nr, d_md);
+  if (p->n_rarcs > 0)
+    EAR_LAUNCH(k_sum_w, (int)std::min<int64_t>(ceil_div(p->n_rarcs, 256), 1024), 256, 0, st)(p->r_w, p->n_rarcs, d_sum);
+  {
+    Readback rb(st);
+    EAR_CUDA_TRY(rb.get(&md, d_md, 4));
+    EAR_CUDA_TRY(rb.get(&wsum, d_sum, 8));
+    EAR_CUDA_TRY(rb.sync());
+  }
+  cudaFreeAsync(d_md, st);
+  // near-far step: 16 mean arc weights (cfg4, simulated: 5x fewer improvements than plain rounds at
+  // about the same round count; smaller steps trade rounds for work)
+  const double mean_w = p->n_rarcs > 0 ? (double)wsum / (double)p->n_rarcs : 1.0;
+  p->r_delta = (uint32_t)std::min(65535.0, std::max(1.0, 16.0 * mean_w));
+  const int K = md <= 4 ? 4 : md <= 8 ? 8 : md <= 12 ? 12 : md <= 16 ? 16 : 0;
+  if (K == 0) return EAR_OK;
+  EAR_CUDA_TRY(cudaMallocAsync((void **)&p->r_ell16, sizeof(uint32_t) * (size_t)K * nr, st));
+  EAR_LAUNCH(k_build_ell16, (int)std::min<int64_t>(ceil_div(nr, 256), 4096), 256, 0, st)(
+      p->r_rowptr, p->r_col, p->r_w, nr, K, p->r_ell16);
+  p->r_k16 = K;
+  return EAR_OK;
+}
+
+// 256 threads per source (512 measured slower in every u16 case: idle warps per round)
+constexpr int SSSP16_NT = 256;
+constexpr int SSSP16_MAX_CTAS = 2048 / SSSP16_NT;
+// shared memory of one source: the row (L entries of db bytes), two lists (cap u16 each), three bitmaps
+static int sssp16_smem(int L, int cap, int db) { return db * L + 4 * cap + 12 * ((L + 31) / 32); }
+
+template <int NTS, int K, typename DistT, typename OutT>
+static ear_status_t sssp16_launch(ear_plan_s *p, OutT *out, int64_t ldo, int32_t L, int32_t row0, int32_t rows,
+                                  const int32_t *trows, int cap, int smem, int32_t *counter, int32_t *sat,
+                                  unsigned long long *d_stats, cudaStream_t st) {
+  constexpr int J = 2;
+  auto kern = k_sssp16<NTS, K, J, DistT, OutT>;
+  EAR_CUDA_TRY(smem_attr((const void *)kern, smem));
+  int per_sm = 1;
+  EAR_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, NTS, smem));
+  const int64_t grid = std::min<int64_t>(rows, (int64_t)num_sms() * std::max(per_sm, 1));
+  int s = prof_begin(PK_SSSP, st);
+  uint32_t delta = p->r_delta;
+  if (const char *e = getenv("EAR_SSSP_DELTA")) delta = atoi(e) > 0 ? (uint32_t)atoi(e) : 0xFFFFFFFFu;   // lab knob
+  EAR_LAUNCH(kern, (unsigned)grid, NTS, smem, st)(reinterpret_cast<const uint4 *>(p->r_ell16), p->n_reduced, L, out,
+                                                  ldo, row0, rows, trows, cap, delta, counter, sat, d_stats);
+  prof_end(s, st, (double)rows * (double)p->n_rarcs);
+  if (d_stats) {
+    unsigned long long h[2];
+    EAR_CUDA_TRY(cudaMemcpyAsync(h, d_stats, 16, cudaMemcpyDeviceToHost, st));
+    EAR_CUDA_TRY(cudaStreamSynchronize(st));
+    fprintf(stderr, "[sssp16 NT=%d K=%d dist=u%d cap=%d smem=%d] grid=%lld per_sm=%d rows=%d rounds=%.1f/source improve=%.0f/source\n",
+            NTS, K, (int)(8 * sizeof(DistT)), cap, smem, (long long)grid, per_sm, rows, (double)h[0] / rows,
+            (double)h[1] / rows);
+  }
+  EAR_CUDA_TRY(cudaGetLastError());
+  return EAR_OK;
+}
+
+template <int NTS, typename DistT, typename OutT>
+static ear_status_t sssp16_dispatch(ear_plan_s *p, OutT *out, int64_t ldo, int32_t L, int32_t row0, int32_t rows,
+                                    const int32_t *trows, int cap, int smem, int32_t *counter, int32_t *sat,
+                                    unsigned long long *d_stats, cudaStream_t st) {
+  switch (p->r_k16) {
+    case 4: return sssp16_launch<NTS, 4, DistT, OutT>(p, out, ldo, L, row0, rows, trows, cap, smem, counter, sat, d_stats, st);
+    case 8: return sssp16_launch<NTS, 8, DistT, OutT>(p, out, ldo, L, row0, rows, trows, cap, smem, counter, sat, d_stats, st);
+    case 12: return sssp16_launch<NTS, 12, DistT, OutT>(p, out, ldo, L, row0, rows, trows, cap, smem, counter, sat, d_stats, st);
+    default: return sssp16_launch<NTS, 16, DistT, OutT>(p, out, ldo, L, row0, rows, trows, cap, smem, counter, sat, d_stats, st);
+  }
+}
+
+// rows [row0, row0 + rows) (or the tile rows listed in trows) into out (u16 or int32, ldo), row length L
+// (a multiple of 8, >= N_r); *applied = false when the route does not apply or a distance saturated
+template <typename OutT>
+static ear_status_t sssp16_rows(ear_plan_s *p, OutT *out, int64_t ldo, int32_t L, int32_t row0, int32_t rows,
+                                const int32_t *trows, bool *applied, cudaStream_t st) {
+  *applied = false;
+  EAR_TRY(ell16_prepare(p, st));
+  if (p->r_k16 <= 0 || L % 8 != 0 || L < p->n_reduced || L >= 0xFFFF) return EAR_OK;
+  int dev = 0, max_smem = 0;
+  EAR_CUDA_TRY(cudaGetDevice(&dev));
+  EAR_CUDA_TRY(cudaDeviceGetAttribute(&max_smem, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev));
+  int per_sm_smem = 0;
+  EAR_CUDA_TRY(cudaDeviceGetAttribute(&per_sm_smem, cudaDevAttrMaxSharedMemoryPerMultiprocessor, dev));
+  // list capacity: as large as lets the most sources share an SM (a near-far frontier of the paper's
+  // sparse reduced graphs stays well below 1k), never below 256; 1 KB per CTA is the driver's, 256 B
+  // the kernel's static shared memory
+  auto fit = [&](int db, int *cap_out) {
+    for (int per = SSSP16_MAX_CTAS; per >= 1; --per) {
+      const int budget = std::min(max_smem, per_sm_smem / per - 1024 - 256);
+      const int c = ((budget - sssp16_smem(L, 0, db)) / 4) & ~7;
+      if (c >= 256) {
+        *cap_out = std::min(c, 4096);
+        return per;
+      }
+    }
+    return 0;
+  };
+  // the row as u32 (one ATOMS.MIN per relaxation) when four sources still share an SM, else the row
+  // type that fits more of them (u16: 16-bit CAS relaxations, half the bytes) -- measured, cfg2 u32 4.8
+  // vs 5.9 ms, cfg3_f60 u16 29.7 vs 31.7 ms, cfg4 u16 136 vs 199 ms
+  int cap4 = 0, cap2 = 0;
+  const int per4 = fit(4, &cap4), per2 = fit(2, &cap2);
+  int db = per4 >= 4 || per4 >= per2 ? 4 : 2;
+  if (const char *e = getenv("EAR_SSSP16_DIST")) db = atoi(e) == 2 ? 2 : atoi(e) == 4 && per4 > 0 ? 4 : db;   // lab
+  int cap = db == 4 ? cap4 : cap2;
+  if (cap == 0) return EAR_OK;
+  if (const char *e = getenv("EAR_SSSP16_CAP")) cap = std::max(16, std::min(cap, atoi(e) & ~7));   // test knob: overflow
+  const int smem = sssp16_smem(L, cap, db);
+  if (rows <= 0) { *applied = true; return EAR_OK; }
+  int32_t *ws = nullptr;
+  EAR_CUDA_TRY(cudaMallocAsync((void **)&ws, 8, st));
+  EAR_CUDA_TRY(dev_memset(ws, 0, 8, st));
+  static unsigned long long *d_stats = nullptr;
+  static const bool want_stats = getenv("EAR_SSSP_STATS") != nullptr;
+  if (want_stats && !d_stats) EAR_CUDA_TRY(cudaMalloc((void **)&d_stats, 16));
+  if (want_stats) EAR_CUDA_TRY(dev_memset(d_stats, 0, 16, st));
+  unsigned long long *stt = want_stats ? d_stats : nullptr;
+  ear_status_t s = EAR_OK;
+  if (db == 4) {
+    s = sssp16_dispatch<SSSP16_NT, uint32_t>(p, out, ldo, L, row0, rows, trows, cap, smem, ws, ws + 1, stt, st);
+  } else {
+    s = sssp16_dispatch<SSSP16_NT, uint16_t>(p, out, ldo, L, row0, rows, trows, cap, smem, ws, ws + 1, stt, st);
+  }
+  int32_t h_sat = 1;
+  if (s == EAR_OK) {
+    Readback rb(st);
+    cudaError_t e = rb.get(&h_sat, ws + 1, 4);
+    if (e == cudaSuccess) e = rb.sync();
+    if (e != cudaSuccess) { set_error("sssp16: %s", cudaGetErrorString(e)); s = EAR_ECUDA; }
+  }
+  cudaFreeAsync(ws, st);
+  if (s == EAR_OK) *applied = h_sat == 0;
+  return s;
+}
+
+ear_status_t sssp_rows16(ear_plan_s *p, uint16_t *D16, int64_t ld16, bool *applied, cudaStream_t st) {
+  const int32_t L = (int32_t)round_up(std::max(p->n_reduced, 1), 8);
+  if (ld16 < L) { *applied = false; return EAR_OK; }
+  return sssp16_rows<uint16_t>(p, D16, ld16, L, 0, p->n_reduced, nullptr, applied, st);
+}
+
 // Rows [row0, row0 + rows) of D (row-major, ldd) by per-source Bellman-Ford on G^r.
 ear_status_t sssp_rows(ear_plan_s *p, int32_t *D, int64_t ldd, int32_t Np, int32_t row0, int32_t rows,
                        const int32_t *trows,
                        cudaStream_t st) {
   EAR_TRY(sssp_prepare(p, st));
   if (rows <= 0) return EAR_OK;
+  static const bool u16_off = [] {
+    const char *e = getenv("EAR_SSSP16");   // 0: the int32 kernels (A/B)
+    return e && atoi(e) == 0;
+  }();
+  if (!u16_off && rows > 1) {   // (one row: the packed FW's precheck -- latency, not throughput)
+    bool applied = false;
+    EAR_TRY(sssp16_rows<int32_t>(p, D, ldd, Np, row0, rows, trows, &applied, st));
+    if (applied) return EAR_OK;
+  }
   const int W = (Np + 31) / 32;
   static unsigned long long *d_stats = nullptr;
   static const bool want_stats = getenv("EAR_SSSP_STATS") != nullptr;

@@ -1,0 +1,16 @@
+cd $GRAFT_REPO_ROOT
+mkdir -p gpurun_out
+T=${TAG:-r02s}
+timeout 900 python -m pytest tests/test_sssp16_gpu.py -q -x -p no:cacheprovider > gpurun_out/${T}_sssp16_tests.txt 2>&1; echo "sssp16 tests rc=$?"; tail -n 2 gpurun_out/${T}_sssp16_tests.txt
+EAR_SSSP16_DIST=2 timeout 900 python -m pytest tests/test_sssp16_gpu.py -q -x -p no:cacheprovider > gpurun_out/${T}_sssp16_tests_u16.txt 2>&1; echo "sssp16 tests (u16 rows) rc=$?"; tail -n 2 gpurun_out/${T}_sssp16_tests_u16.txt
+timeout 900 python -m pytest tests/test_parity_gpu.py -q -x -p no:cacheprovider -k "sssp" > gpurun_out/${T}_sssp_parity.txt 2>&1; echo "sssp parity rc=$?"; tail -n 1 gpurun_out/${T}_sssp_parity.txt
+for d in 4 2; do for nt in 256 512; do
+  echo "== dist $d nt $nt"
+  EAR_SSSP16_DIST=$d EAR_SSSP16_NT=$nt EAR_SSSP_STATS=1 timeout 600 python tools/time_sssp.py cfg4 --reps 1 --no-full --no-fw 2>&1 | grep -E "^\[sssp16" | sort -u
+  EAR_SSSP16_DIST=$d EAR_SSSP16_NT=$nt timeout 600 python tools/time_sssp.py cfg2 cfg3_f60 cfg4 --reps 3 --no-full --no-fw --out gpurun_out/${T}_lab_d${d}_nt${nt}.jsonl 2>&1 | tail -n 3
+done; done
+for dl in 460 920 3680 7360 0; do
+  echo "== delta $dl"
+  EAR_SSSP_DELTA=$dl EAR_SSSP_STATS=1 timeout 600 python tools/time_sssp.py cfg4 --reps 1 --no-full --no-fw 2>&1 | grep -E "^\[sssp16" | sort -u
+  EAR_SSSP_DELTA=$dl timeout 600 python tools/time_sssp.py cfg4 --reps 3 --no-full --no-fw --out gpurun_out/${T}_delta${dl}.jsonl 2>&1 | tail -n 1
+done
