@@ -4,17 +4,19 @@
     python bench.py [--gpus N] [--steps K] [--warmup W] [--config cfg4] [--impl ours|reference]
 
 One step = one pass of the whole hot path over the workload: apsp_full =
-Reduce(G) chain contraction -> blocked min-plus FW on G^r -> ear expansion of this rank's rows of the
-N x N int32 matrix, graph already resident in HBM.  By default (--phase2 bcc) Phase II runs the FW on
-the biconnected pieces of G^r and joins them through the articulation points (paper sec. 2.2,
-P:119-131); --phase2 fw runs one FW over all of G^r, --phase2 sssp the per-source SSSP.  For N > 1 GPUs (torchrun, one process per GPU)
-the FW is row-block sharded with a per-round NCCL pivot broadcast and every rank expands its own row
+Reduce(G) chain contraction -> Phase II on G^r -> ear expansion of this rank's rows of the N x N int32
+matrix, graph already resident in HBM.  By default (--phase2 bcc_sssp) Phase II splits G^r into its
+biconnected pieces (paper sec. 2.2), reduces every big piece again and solves it by
+the paper's own per-source SSSP (near-far rounds on u16 shared-memory rows), joining the pieces
+through the articulation points; --phase2 bcc solves the pieces by the blocked min-plus FW, --phase2 fw
+runs one FW over all of G^r, --phase2 sssp the SSSP over all of G^r.  For N > 1 GPUs (torchrun, one
+process per GPU) the largest piece's rows are split over the ranks and every rank expands its own row
 block; the total work is fixed (strong scaling).  Timing: W untimed warm-up steps, then exactly K
-steps between barrier + synchronize, CUDA events on the launching stream, max over ranks.  D (3.6 GB)
-and the output (40 GB) are far larger than L2, so no flush is needed between steps.
+steps between barrier + synchronize, CUDA events on the launching stream, max over ranks.  The output
+(40 GB) is far larger than L2, so no flush is needed between steps.
 
-Rank 0 prints one JSON line.  Extra keys: roofline (dominant kernel = FW phase-3 min-plus tile
-kernel, ALU bound), roofline_expand (HBM bound), cpu_baseline (the CPU oracle on a bounded sample,
+Rank 0 prints one JSON line.  Extra keys: roofline (dominant kernel: the per-source SSSP, or the FW
+phase-3 min-plus tile kernel on the FW routes), roofline_expand (HBM bound), cpu_baseline (the CPU oracle on a bounded sample,
 rank 0 at N = 1 only), e2e (the same metric through the host-buffer C-ABI calls with every step's
 H2D edge upload and D2H copy of the output rows: by default K jobs of apsp_full_host_async pipelined one
 deep -- job i+1's Phases I-II overlap job i's expansion and row copies -- into two pinned output buffers;
@@ -270,9 +272,10 @@ def run_ours(args, rank, world, local_rank):
     plan.destroy()
     stream = torch.cuda.current_stream(dev)
 
-    flags = {"fw": 0, "sssp": ea.FLAG_SSSP, "bcc": ea.FLAG_BCC}[args.phase2] | (ea.FLAG_FW32 if args.fw32 else 0)
+    flags = {"fw": 0, "sssp": ea.FLAG_SSSP, "bcc": ea.FLAG_BCC, "bcc_sssp": ea.FLAG_BCC | ea.FLAG_SSSP}[args.phase2] \
+        | (ea.FLAG_FW32 if args.fw32 else 0)
     bcc = None
-    if args.phase2 == "bcc":
+    if args.phase2 in ("bcc", "bcc_sssp"):
         pb = ea.ear_decompose(g.n, src, dst, w, flags=flags)
         if world == 1 and not args.no_alt:   # one untimed Phase II: the re-reduction counts of a solve
             Dp = ea.alloc_D(pb)
@@ -367,14 +370,24 @@ def run_ours(args, rank, world, local_rank):
     K = args.steps
     # main-stream FW time; the lookahead's side-stream pivot work overlaps phase 3 (fw_side_overlapped)
     fw_ms = prof["fw_init_ms"] + prof["fw_phase1_ms"] + prof["fw_phase2_ms"] + prof["fw_phase3_ms"] + prof["fw16_conv_ms"]
-    if args.phase2 == "sssp":   # the dominant kernel is the per-source SSSP (latency / L2-atomic bound)
+    if args.phase2 in ("sssp", "bcc_sssp"):   # the dominant kernel is the per-source SSSP
+        # algorithmic work: Dijkstra's relaxation count, every arc of the solved graph once per source;
+        # peak: each relaxation needs at least one shared-memory load of d(u) and an SM serves one
+        # conflict-free 32-lane shared load per clock (the kernel is bound by its round
+        # latency, far below this)
         sssp_ms = prof["sssp_ms"]
-        roofline = {"bound": "latency", "kernel": "k_sssp_bf (Phase II by per-source SSSP)",
-                    "achieved": prof["sssp_arcs"] / (sssp_ms / 1e3) / 1e9 if sssp_ms > 0 else 0.0,
-                    "peak": None, "unit": "G arc-relaxations/s (one pass over G^r per source)", "frac": None,
-                    "traffic": ncu_traffic("k_sssp_bf", args.config),
-                    "avg_launch_ms": sssp_ms / max(prof["sssp_launches"], 1),
-                    "note": "label-correcting Bellman-Ford per source; no arithmetic roofline applies"}
+        n_ss = max(prof["sssp_launches"], 1)
+        ach = prof["sssp_arcs"] / (sssp_ms / 1e3) / 1e9 if sssp_ms > 0 else 0.0
+        peak_relax = SM_COUNT * 32 * sm_max * 1e6 / 1e9
+        roofline = {"bound": "alu", "kernel": "k_sssp16 (Phase II: per-source near-far SSSP on the reduced pieces)",
+                    "achieved": ach, "peak": peak_relax, "unit": "G relaxations/s", "frac": ach / peak_relax,
+                    "traffic": ncu_traffic("k_sssp16", args.config), "avg_launch_ms": sssp_ms / n_ss,
+                    "relaxations_per_launch": prof["sssp_arcs"] / n_ss,
+                    "peak_basis": f"{SM_COUNT} SMs x 32 shared-memory lanes/clk x {sm_max:.0f} MHz: one conflict-free "
+                                  "load of d(u) per relaxation (an upper bound; the kernel is round-latency bound, "
+                                  "DESIGN.md 6b)"}
+        if clocks.get("sm_mhz"):
+            roofline["frac_at_run_clock"] = ach / (SM_COUNT * 32 * clocks["sm_mhz"] * 1e6 / 1e9)
     phases = {"decompose": prof["decompose_ms"] / K, "fw": fw_ms / K, "sssp": prof["sssp_ms"] / K, "fw_phase1": prof["fw_phase1_ms"] / K,
               "fw_phase2": prof["fw_phase2_ms"] / K, "fw_phase3": p3_ms / K, "comm": prof["comm_ms"] / K,
               "expand": ex_ms / K, "same_chain": prof["same_chain_ms"] / K,
@@ -391,7 +404,7 @@ def run_ours(args, rank, world, local_rank):
     alt = None
     if world == 1 and not args.no_alt:
         alt = {"note": "Phase II only (D of G^r), one timed call after a warm-up call; --phase2 X times the full step"}
-        for name, fl in (("fw", 0), ("sssp", ea.FLAG_SSSP), ("bcc", ea.FLAG_BCC)):
+        for name, fl in (("fw", 0), ("sssp", ea.FLAG_SSSP), ("bcc", ea.FLAG_BCC), ("bcc_sssp", ea.FLAG_BCC | ea.FLAG_SSSP)):
             if name == args.phase2:
                 continue
             p2 = ea.ear_decompose(g.n, src, dst, w, flags=fl)
@@ -490,7 +503,9 @@ def run_ours(args, rank, world, local_rank):
     if rank == 0:
         line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": K, "warmup": args.warmup,
                 "ms_per_step": ms_max / K, "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
-                "dtype": "int32" if prof["fw16_used"] == 0 else "int32 (FW: packed u16x2, exact below 0x7FFF)",
+                "dtype": ("int32 (SSSP: u16 shared-memory rows, exact below 0xFFFF; int32 fallback)"
+                          if args.phase2 in ("sssp", "bcc_sssp") else
+                          "int32" if prof["fw16_used"] == 0 else "int32 (FW: packed u16x2, exact below 0x7FFF)"),
                 "data": "synthetic (seeded generator, spatially coherent labels)",
                 "fw16": {"used": int(prof["fw16_used"]) // K, "fallbacks": int(prof["fw16_fallbacks"]) // K},
                 "config": {"workload": WORKLOADS.get(args.config, args.config), "name": args.config,
@@ -523,9 +538,10 @@ def main():
     ap.add_argument("--config", default="cfg4")
     ap.add_argument("--seed", type=int, default=0)
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
-    ap.add_argument("--phase2", choices=["bcc", "fw", "sssp"], default="bcc",
-                    help="Phase II: blocked FW on the biconnected pieces of G^r (paper sec. 2.2, default), "
-                         "blocked FW on all of G^r, or per-source SSSP (SURVEY 8.f NEXT 2)")
+    ap.add_argument("--phase2", choices=["bcc_sssp", "bcc", "fw", "sssp"], default="bcc_sssp",
+                    help="Phase II: the biconnected pieces of G^r (paper sec. 2.2) each reduced again and solved by "
+                         "per-source SSSP (the paper's own Phase II, P:101; default), the same pieces by blocked FW, "
+                         "blocked FW on all of G^r, or per-source SSSP on all of G^r")
     ap.add_argument("--fw32", action="store_true", help="int32 FW throughout (EAR_FLAG_FW32)")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=4)

@@ -56,7 +56,9 @@ enum {
   EAR_FLAG_BCC = 4,         /* Phase II by biconnected pieces (paper sec. 2.2; SURVEY 8.f
                                NEXT 3): FW on the largest block of every component and on the pieces
                                hanging off it, joined through the articulation points; same D
-                               bit for bit.  Exclusive with EAR_FLAG_SSSP. */
+                               bit for bit.  With EAR_FLAG_SSSP too, every big piece is reduced again
+                                and its reduced graph solved by the per-source SSSP instead of
+                               the FW (the bench's route: O(n m) work per piece instead of O(n^3)). */
   EAR_FLAG_FW32 = 8         /* single-GPU FW: skip the packed 16-bit attempt and run int32 throughout.
                                By default the FW first runs on a copy of D capped at 0x7FFF with two
                                min-plus per VIADDMNMX.U16x2 (exact for every distance < 0x7FFF, see

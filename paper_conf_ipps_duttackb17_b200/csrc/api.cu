@@ -106,10 +106,6 @@ ear_status_t ear_decompose(int32_t n, int64_t m, const int32_t *d_src, const int
     set_error("ear_decompose: bad sizes n=%d m=%lld", n, (long long)m);
     return EAR_EINVAL;
   }
-  if ((flags & EAR_FLAG_SSSP) && (flags & EAR_FLAG_BCC)) {
-    set_error("ear_decompose: EAR_FLAG_SSSP and EAR_FLAG_BCC are exclusive");
-    return EAR_EINVAL;
-  }
   ear_plan_s *p = new ear_plan_s;
   cudaGetDevice(&p->device);
   int sp = prof_begin(PK_DECOMPOSE, (cudaStream_t)stream);
@@ -179,8 +175,8 @@ ear_status_t apsp_reduced(ear_plan_t p, int32_t *d_D, int64_t ldd, ear_comm_t co
   }
   cudaStream_t st = (cudaStream_t)stream;
   if (!comm) {
-    if (p->flags & EAR_FLAG_SSSP) return sssp_rows(p, d_D, ldd, Np, 0, Np, nullptr, st);
     if (p->flags & EAR_FLAG_BCC) return bcc_solve(p, nullptr, d_D, ldd, Np, 0, Np, nullptr, st);
+    if (p->flags & EAR_FLAG_SSSP) return sssp_rows(p, d_D, ldd, Np, 0, Np, nullptr, st);
     EAR_TRY(fw_init_D(p, d_D, ldd, Np, 0, Np, st));
     const bool allow16 = !(p->flags & EAR_FLAG_FW32);
     const int32_t *lab = nullptr;
@@ -193,10 +189,10 @@ ear_status_t apsp_reduced(ear_plan_t p, int32_t *d_D, int64_t ldd, ear_comm_t co
   int32_t *d_rows = nullptr, nown = 0;
   EAR_TRY(shard_rows_device(nt, P, comm->rank, &d_rows, &nown, st));
   ear_status_t s = EAR_OK;
-  if (p->flags & EAR_FLAG_SSSP) {   // every rank its own rows: no exchange in Phase II
-    s = sssp_rows(p, d_D, ldd, Np, 0, nown * TILE, d_rows, st);
-  } else if (p->flags & EAR_FLAG_BCC) {   // largest piece sharded, owned rows composed
+  if (p->flags & EAR_FLAG_BCC) {   // largest piece sharded, owned rows composed
     s = bcc_solve(p, comm, d_D, ldd, Np, 0, nown * TILE, d_rows, st);
+  } else if (p->flags & EAR_FLAG_SSSP) {   // every rank its own rows: no exchange in Phase II
+    s = sssp_rows(p, d_D, ldd, Np, 0, nown * TILE, d_rows, st);
   } else {
     std::vector<int32_t> rows(nown);
     if (nown > 0) {
@@ -329,7 +325,7 @@ static ear_status_t solve_rows(ear_plan_s *p, int32_t row_begin, int32_t row_end
       k.D16 = nullptr;
     }
   }
-  if (!comm && (p->flags & EAR_FLAG_SSSP) && u16_ok && xp_applicable(p, st)) {
+  if (!comm && (p->flags & EAR_FLAG_SSSP) && !(p->flags & EAR_FLAG_BCC) && u16_ok && xp_applicable(p, st)) {
     // per-source SSSP straight into u16 rows: no int32 D, no narrowing pass
     k.ld16 = xp_row_stride(p);
     EAR_CUDA_TRY(cudaMallocAsync((void **)&k.D16, sizeof(uint16_t) * (size_t)p->n_reduced * k.ld16, st));

@@ -742,9 +742,13 @@ static ear_status_t reduce_solve(const ear_plan_s *p, int32_t n, int64_t m, cons
   int sr = prof_begin(PK_REREDUCE, st);
   ear_status_t s = decompose(n, m, u, v, w, p->flags & EAR_FLAG_FW32, st, q);
   prof_end(sr, st, 0);
-  // worth it when the FW runs on fewer 128-tiles (same tile count: same FW work, plus the expansion)
+  // worth it when the FW runs on fewer 128-tiles (same tile count: same FW work, plus the expansion);
+  // pieces solved by SSSP (EAR_FLAG_SSSP) always take the top level -- its plan is what the SSSP runs
+  // on -- and a deeper one when it removes vertices
+  const bool by_sssp = (p->flags & EAR_FLAG_SSSP) != 0;
   const int64_t unit = (int64_t)TILE * (comm ? comm->nranks : 1);
-  const bool worth = s == EAR_OK && round_up(std::max<int64_t>(q->n_reduced, 1), unit) < round_up(n, unit);
+  const bool worth = s == EAR_OK && (by_sssp ? depth == 0 || q->n_reduced < n
+                                             : round_up(std::max<int64_t>(q->n_reduced, 1), unit) < round_up(n, unit));
   if (!worth) {
     cudaStreamSynchronize(st);
     plan_free(q);
@@ -767,15 +771,26 @@ static ear_status_t reduce_solve(const ear_plan_s *p, int32_t n, int64_t m, cons
                      levels, n_last);
   if (s == EAR_OK && !inner) {
     if (!comm) {
-      s = fw_init_D(q, D, Np, Np, 0, Np, st);
-      if (s == EAR_OK) s = fw_single(D, Np, Np, st, nullptr, q->n_reduced, allow16, q);   // connected
+      if (by_sssp) {
+        s = sssp_rows(q, D, Np, Np, 0, Np, nullptr, st);
+      } else {
+        s = fw_init_D(q, D, Np, Np, 0, Np, st);
+        if (s == EAR_OK) s = fw_single(D, Np, Np, st, nullptr, q->n_reduced, allow16, q);   // connected
+      }
     } else {
       const std::vector<int32_t> own = shard_rows(Np / TILE, P, comm->rank);
       int32_t *S = nullptr;   // the owned rows live in this rank's exchange window (read there by the gather)
       s = fw_shard_buffer(comm, Np, st, &S);
-      for (size_t j = 0; j < own.size() && s == EAR_OK; ++j)
-        s = fw_init_D(q, S + (int64_t)j * TILE * Np, Np, Np, own[j] * TILE, TILE, st);
-      if (s == EAR_OK) s = fw_sharded_auto(S, Np, Np, comm, nullptr, q->n_reduced, allow16, st, q);
+      if (by_sssp) {   // every rank its own tile rows, no exchange until the gather
+        int32_t *d_rows = nullptr, nown = 0;
+        if (s == EAR_OK) s = shard_rows_device(Np / TILE, P, comm->rank, &d_rows, &nown, st);
+        if (s == EAR_OK) s = sssp_rows(q, S, Np, Np, 0, nown * TILE, d_rows, st);
+        if (d_rows) cudaFreeAsync(d_rows, st);
+      } else {
+        for (size_t j = 0; j < own.size() && s == EAR_OK; ++j)
+          s = fw_init_D(q, S + (int64_t)j * TILE * Np, Np, Np, own[j] * TILE, TILE, st);
+        if (s == EAR_OK) s = fw_sharded_auto(S, Np, Np, comm, nullptr, q->n_reduced, allow16, st, q);
+      }
       if (s == EAR_OK) s = fw_sharded_gather(S, Np, Np, D, Np, comm, st);
     }
   }

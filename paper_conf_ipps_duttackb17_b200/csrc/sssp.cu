@@ -417,7 +417,7 @@ __device__ __forceinline__ bool sssp_lower(DistT *d, uint32_t nd, uint32_t cur) 
 }
 
 template <int NTS, int K, int J, typename DistT, typename OutT>
-__global__ void __launch_bounds__(NTS) k_sssp16(const uint4 *__restrict__ ell, int32_t nr, int32_t L, OutT *out,
+__global__ void __launch_bounds__(NTS, 3) k_sssp16(const uint4 *__restrict__ ell, int32_t nr, int32_t L, OutT *out,
                                                int64_t ldo, int32_t src0, int32_t nsrc, const int32_t *trows, int cap,
                                                uint32_t delta, int32_t *counter, int32_t *sat,
                                                unsigned long long *stats) {
@@ -519,7 +519,7 @@ __global__ void __launch_bounds__(NTS) k_sssp16(const uint4 *__restrict__ ell, i
               for (int k = 0; k < K; ++k) {
                 const uint4 q = e[j][k / 4];
                 const uint32_t a = (k & 3) == 0 ? q.x : (k & 3) == 1 ? q.y : (k & 3) == 2 ? q.z : q.w;
-                if (!__any_sync(0xFFFFFFFFu, (a & 0xFFFFu) != 0xFFFFu)) break;
+                if (!__any_sync(0xFFFFFFFFu, (a & 0xFFFFu) != 0xFFFFu)) break;   // padding from here on
                 const bool push = relax(dv, a);
                 const unsigned bal = __ballot_sync(0xFFFFFFFFu, push);
                 if (push) {
@@ -857,7 +857,7 @@ template <int NTS, int K, typename DistT, typename OutT>
 static ear_status_t sssp16_launch(ear_plan_s *p, OutT *out, int64_t ldo, int32_t L, int32_t row0, int32_t rows,
                                   const int32_t *trows, int cap, int smem, int32_t *counter, int32_t *sat,
                                   unsigned long long *d_stats, cudaStream_t st) {
-  constexpr int J = 2;
+  constexpr int J = 2;   // two 32-vertex tasks per warp when the frontier is wide (their ELL loads overlap)
   auto kern = k_sssp16<NTS, K, J, DistT, OutT>;
   EAR_CUDA_TRY(smem_attr((const void *)kern, smem));
   int per_sm = 1;
@@ -868,7 +868,9 @@ static ear_status_t sssp16_launch(ear_plan_s *p, OutT *out, int64_t ldo, int32_t
   if (const char *e = getenv("EAR_SSSP_DELTA")) delta = atoi(e) > 0 ? (uint32_t)atoi(e) : 0xFFFFFFFFu;   // lab knob
   EAR_LAUNCH(kern, (unsigned)grid, NTS, smem, st)(reinterpret_cast<const uint4 *>(p->r_ell16), p->n_reduced, L, out,
                                                   ldo, row0, rows, trows, cap, delta, counter, sat, d_stats);
-  prof_end(s, st, (double)rows * (double)p->n_rarcs);
+  // algorithmic work: one relaxation per arc per (real) source -- Dijkstra's count; padding sources are free
+  const int64_t real = trows ? rows : std::max<int64_t>(0, std::min<int64_t>(rows, (int64_t)p->n_reduced - row0));
+  prof_end(s, st, (double)real * (double)p->n_rarcs);
   if (d_stats) {
     unsigned long long h[2];
     EAR_CUDA_TRY(cudaMemcpyAsync(h, d_stats, 16, cudaMemcpyDeviceToHost, st));

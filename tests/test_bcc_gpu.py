@@ -232,10 +232,51 @@ def test_bcc_degenerate(pkg, case):
     assert_exact(run_full(pkg, g, pkg.FLAG_BCC), oracle.apsp(g.n, g.src, g.dst, g.w), case)
 
 
-def test_bcc_flags_exclusive(pkg):
-    g = gg.cycle(5, seed=1)
-    with pytest.raises(pkg.EarError, match="EINVAL"):
-        pkg.ear_decompose(g.n, dev(g.src), dev(g.dst), dev(g.w), flags=pkg.FLAG_BCC | pkg.FLAG_SSSP)
+# ------------------------------------------------------------------------------ blocks solved by SSSP
+# EAR_FLAG_BCC | EAR_FLAG_SSSP: the block structure of sec. 2.2 with every big piece reduced
+# again and its reduced graph solved by the paper's per-source SSSP instead of the FW.
+@pytest.mark.parametrize("seed", range(10))
+def test_bcc_sssp_block_trees(pkg, seed):
+    g = gg.block_tree(40 + seed, n_target=300 + 500 * seed, big=200 * (seed % 4))
+    assert_exact(run_full(pkg, g, pkg.FLAG_BCC | pkg.FLAG_SSSP), oracle.apsp(g.n, g.src, g.dst, g.w),
+                 f"bcc+sssp block tree {seed}")
+
+
+@pytest.mark.parametrize("seed", range(8))
+def test_bcc_sssp_corner_cases(pkg, seed):
+    g = gg.corner_cases(7000 + seed, n_target=30 + 25 * seed)
+    assert_exact(run_full(pkg, g, pkg.FLAG_BCC | pkg.FLAG_SSSP), oracle.apsp(g.n, g.src, g.dst, g.w),
+                 f"bcc+sssp corner {seed}")
+
+
+@pytest.mark.parametrize("seed", range(2))
+def test_bcc_sssp_rereduced_pieces(pkg, seed):
+    g = decorated_grid(24 + 4 * seed, 0.3 + 0.1 * seed, seed)
+    assert_exact(run_full(pkg, g, pkg.FLAG_BCC | pkg.FLAG_SSSP), oracle.apsp(g.n, g.src, g.dst, g.w),
+                 f"bcc+sssp rereduce {seed}")
+
+
+@pytest.mark.parametrize("name", ["cfg2", "block"])
+def test_bcc_sssp_D_equals_fw_D(pkg, name):
+    g = gg.block_tree(7, n_target=8000, big=1500) if name == "block" else gg.config(name)
+    p1 = pkg.ear_decompose(g.n, dev(g.src), dev(g.dst), dev(g.w))
+    p2 = pkg.ear_decompose(g.n, dev(g.src), dev(g.dst), dev(g.w), flags=pkg.FLAG_BCC | pkg.FLAG_SSSP)
+    D1, D2 = pkg.alloc_D(p1), pkg.alloc_D(p2)
+    pkg.apsp_reduced(p1, D1)
+    pkg.apsp_reduced(p2, D2)
+    torch.cuda.synchronize()
+    assert torch.equal(D1, D2)
+
+
+def test_bcc_sssp_cfg4_sampled_rows(pkg):
+    """the bench's route at its size: full N x N through apsp_full (u16 compose), sampled rows"""
+    g = gg.config("cfg4")
+    out = pkg.apsp_full(g.n, dev(g.src), dev(g.dst), dev(g.w), flags=pkg.FLAG_BCC | pkg.FLAG_SSSP)
+    rows = np.unique(np.concatenate([[0, g.n - 1], np.random.default_rng(10).choice(g.n, 24, replace=False)]))
+    ref = oracle.apsp_rows(g.n, g.src, g.dst, g.w, rows)
+    assert_exact(out[torch.as_tensor(rows).cuda().long()].cpu().numpy(), ref, "cfg4 bcc+sssp rows")
+    del out
+    torch.cuda.empty_cache()
 
 
 # ------------------------------------------------------------------------------ structure

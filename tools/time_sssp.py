@@ -54,12 +54,18 @@ def main():
             rec["D_equal"] = bool(torch.equal(D, D2))
             del D2, p2
         del D, p
+        p3 = ea.ear_decompose(g.n, src, dst, w, flags=ea.FLAG_BCC | ea.FLAG_SSSP)
+        D3 = ea.alloc_D(p3)
+        rec["reduced_bcc_sssp_ms"] = timed(lambda: ea.apsp_reduced(p3, D3), a.reps)
+        del D3, p3
         torch.cuda.empty_cache()
         if not a.no_full:
             out = torch.empty((g.n, g.n), dtype=torch.int32, device="cuda")
-            for fl, key in ((ea.FLAG_SSSP, "full_sssp_ms"), (ea.FLAG_BCC, "full_bcc_ms")):
+            for fl, key in ((ea.FLAG_SSSP, "full_sssp_ms"), (ea.FLAG_BCC | ea.FLAG_SSSP, "full_bcc_sssp_ms"),
+                            (ea.FLAG_BCC, "full_bcc_ms")):
                 rec[key] = timed(lambda: ea.apsp_full(g.n, src, dst, w, out=out, flags=fl), a.reps)
             rec["full_sssp_entries_per_s"] = g.n * g.n / (rec["full_sssp_ms"] * 1e-3)
+            rec["full_bcc_sssp_entries_per_s"] = g.n * g.n / (rec["full_bcc_sssp_ms"] * 1e-3)
             del out
             torch.cuda.empty_cache()
         print(json.dumps(rec), flush=True)
