@@ -83,6 +83,7 @@ struct ear_plan_s {
   uint32_t *r_ell16 = nullptr;  // u16 route: ELL rows of r_k16 packed arcs (target | min(w, 0xFFFF) << 16)
   int32_t r_k16 = -1;           // 0: the u16 route does not apply (N_r >= 0xFFFF or a degree > 16)
   uint32_t r_delta = 0;         // near-far step of the u16 SSSP (16 x the mean arc weight)
+  uint16_t *r_maxnb = nullptr;  // largest neighbour id per reduced vertex (the SSSP's known-prefix boundary)
   int32_t n_rarcs = 0;
   ear_bcc_s *bcc = nullptr;     // built on first use (EAR_FLAG_BCC, ear_bcc_info)
   int32_t *cc = nullptr;        // [cc_np] connected-component labels of G^r (16-bit FW range check)

@@ -302,7 +302,7 @@ struct Scratch {
 void plan_free(ear_plan_s *p) {
   if (!p) return;
   void *arrs[] = {p->desc, p->tid, p->ear, p->seg_of, p->seg_start, p->seg_vert, p->re_u, p->re_v, p->re_w, p->re_x,
-                  p->r_rowptr, p->r_col, p->r_w, p->r_arcs, p->r_ell16};
+                  p->r_rowptr, p->r_col, p->r_w, p->r_arcs, p->r_ell16, p->r_maxnb};
   for (void *a : arrs)
     if (a) cudaFreeAsync(a, p->stream);
   bcc_free(p->bcc, p->stream);

@@ -420,6 +420,7 @@ template <int NTS, int K, int J, typename DistT, typename OutT>
 __global__ void __launch_bounds__(NTS, 3) k_sssp16(const uint4 *__restrict__ ell, int32_t nr, int32_t L, OutT *out,
                                                int64_t ldo, int32_t src0, int32_t nsrc, const int32_t *trows, int cap,
                                                uint32_t delta, int32_t *counter, int32_t *sat,
+                                               const uint16_t *__restrict__ maxnb, int32_t *done, int32_t *wm,
                                                unsigned long long *stats) {
   constexpr int NW = NTS / 32;
   constexpr uint32_t DINF = sizeof(DistT) == 2 ? 0xFFFFu : 0xFFFFFFFFu;
@@ -432,6 +433,7 @@ __global__ void __launch_bounds__(NTS, 3) k_sssp16(const uint4 *__restrict__ ell
   uint16_t *Lb = reinterpret_cast<uint16_t *>(F + W);                        // [2][NW][S]
   __shared__ int scnt[3][NW], ovf[3], s_item, s_sat;
   __shared__ uint32_t s_min[NW];
+  __shared__ int s_red[NW], s_k;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const uint32_t lt = (1u << lane) - 1u;
   const int wpt = (W + NTS - 1) / NTS, w0 = tid * wpt, w1 = min(W, w0 + wpt);   // owned bitmap words
@@ -442,22 +444,70 @@ __global__ void __launch_bounds__(NTS, 3) k_sssp16(const uint4 *__restrict__ ell
     const int32_t li = s_item;
     if (li >= nsrc) break;
     const int32_t src = trows ? trows[li >> 7] * TILE + (li & (TILE - 1)) : src0 + li;
+    // D is symmetric (G undirected): with `maxnb`, the rows of the finished prefix [0, kmax) of sources
+    // give d(t, src) = D[t][src] exactly.  Those vertices are final; only the ones with a neighbour
+    // >= kmax (maxnb[t] >= kmax) can improve the rest, so they seed the search with the source.
+    int kmax = 0;
+    if (maxnb) {
+      if (tid == 0) s_k = *(volatile int32_t *)wm;
+      __syncthreads();
+      int k = s_k;
+      while (k < li) {   // uniform: the first unfinished row at or after the watermark
+        const int t = k + tid;
+        const bool fin = t < li && *(volatile const int32_t *)(done + t) != 0;
+        const int first = __reduce_min_sync(0xFFFFFFFFu, fin ? 0x7FFFFFFF : min(t, li));
+        if (lane == 0) s_red[warp] = first;
+        __syncthreads();
+        int f = 0x7FFFFFFF;
+#pragma unroll
+        for (int w = 0; w < NW; ++w) f = min(f, s_red[w]);
+        __syncthreads();
+        if (f != 0x7FFFFFFF) { k = f; break; }
+        k += NTS;
+      }
+      kmax = min(k, li);
+      if (tid == 0 && kmax > s_k) atomicMax(wm, kmax);
+      __threadfence();   // acquire: the rows of [0, kmax) are read below
+    }
     for (int i = tid; i < L * (int)sizeof(DistT) / 16; i += NTS)
       reinterpret_cast<uint4 *>(dist)[i] = make_uint4(~0u, ~0u, ~0u, ~0u);
-    for (int w = tid; w < 3 * W; w += NTS) Mb[w] = 0u;   // both list bitmaps and F
+    for (int w = tid; w < 2 * W; w += NTS) Mb[w] = 0u;   // both list bitmaps
     if (tid < 3 * NW) (&scnt[0][0])[tid] = 0;
     if (tid < 3) ovf[tid] = 0;
     if (tid == 0) s_sat = 0;
     __syncthreads();
-    if (tid == 0) {
-      dist[src] = 0;   // a padding source (src >= nr) has no arcs: its row is INF but the diagonal
-      Lb[0] = (uint16_t)src;
-      Mb[src >> 5] = 1u << (src & 31);
-      scnt[0][0] = 1;
+#pragma unroll 4
+    for (int t = tid; t < kmax; t += NTS) {   // column src of the finished rows (L2: written by other CTAs)
+      const uint32_t x = (uint32_t)__ldcg(out + (int64_t)t * ldo + src);
+      dist[t] = (DistT)(x >= 0xFFFFu ? DINF : x);
     }
     __syncthreads();
+    // the far pile starts as {src} + the boundary of the known prefix; round 0 is empty and its advance
+    // (thr 0 -> smallest seed + delta) lists every seed below the first threshold
+    for (int w = w0; w < w1; ++w) {
+      uint32_t f = 0u;
+      const int t0 = w << 5;
+      if (t0 < kmax) {
+        const uint4 *mq = reinterpret_cast<const uint4 *>(maxnb + t0);
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+          const uint4 m4 = __ldg(mq + q);
+          const uint32_t mm[4] = {m4.x, m4.y, m4.z, m4.w};
+#pragma unroll
+          for (int h = 0; h < 8; ++h) {
+            const int b = q * 8 + h, t = t0 + b;
+            const uint32_t nb = (mm[h >> 1] >> ((h & 1) * 16)) & 0xFFFFu;
+            if (t < kmax && nb >= (uint32_t)kmax && dist[t] != (DistT)DINF) f |= 1u << b;
+          }
+        }
+      }
+      if ((src >> 5) == w) f |= 1u << (src & 31);
+      F[w] = f;
+    }
+    if (tid == 0) dist[src] = 0;   // a padding source (src >= nr) has no arcs: its row is INF but the diagonal
+    __syncthreads();
     if (src < nr) {
-      uint32_t thr = delta;   // near-far: only vertices below thr are expanded (uniform)
+      uint32_t thr = 0;   // near-far: only vertices below thr are expanded (uniform)
       for (int r = 0;; ++r) {
         const uint16_t *Lc = Lb + (r & 1) * (NW * S);
         uint16_t *Ln = Lb + ((r + 1) & 1) * (NW * S) + warp * S;   // this warp's segment
@@ -657,6 +707,10 @@ __global__ void __launch_bounds__(NTS, 3) k_sssp16(const uint4 *__restrict__ ell
       }
     }
     __syncthreads();
+    if (maxnb && tid == 0) {   // publish: every thread's row stores precede the flag (barrier + fence)
+      __threadfence();
+      atomicExch(done + li, 1);
+    }
   }
   if (stats) {
     if (tid == 0) atomicAdd(&stats[0], my_rounds);
@@ -669,6 +723,15 @@ __global__ void k_sum_w(const int32_t *w, int32_t A, unsigned long long *sum) {
   for (int64_t a = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; a < A; a += (int64_t)gridDim.x * blockDim.x)
     t += (unsigned long long)w[a];
   atomicAdd(sum, t);
+}
+
+__global__ void k_maxnb16(const int32_t *rowptr, const int32_t *col, int32_t nr, int32_t len, uint16_t *mx) {
+  for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < len; v += (int64_t)gridDim.x * blockDim.x) {
+    int m = 0;
+    if (v < nr)
+      for (int a = rowptr[v]; a < rowptr[v + 1]; ++a) m = max(m, col[a]);
+    mx[v] = (uint16_t)m;
+  }
 }
 
 __global__ void k_build_ell16(const int32_t *rowptr, const int32_t *col, const int32_t *w, int32_t nr, int K,
@@ -840,6 +903,10 @@ static ear_status_t ell16_prepare(ear_plan_s *p, cudaStream_t st) {
   p->r_delta = (uint32_t)std::min(65535.0, std::max(1.0, 16.0 * mean_w));
   const int K = md <= 4 ? 4 : md <= 8 ? 8 : md <= 12 ? 12 : md <= 16 ? 16 : 0;
   if (K == 0) return EAR_OK;
+  const int32_t lm = (int32_t)round_up(nr, 64);   // read in whole 32-vertex words by the kernel
+  EAR_CUDA_TRY(cudaMallocAsync((void **)&p->r_maxnb, sizeof(uint16_t) * (size_t)lm, st));
+  EAR_LAUNCH(k_maxnb16, (int)std::min<int64_t>(ceil_div(lm, 256), 4096), 256, 0, st)(p->r_rowptr, p->r_col, nr, lm,
+                                                                                   p->r_maxnb);
   EAR_CUDA_TRY(cudaMallocAsync((void **)&p->r_ell16, sizeof(uint32_t) * (size_t)K * nr, st));
   EAR_LAUNCH(k_build_ell16, (int)std::min<int64_t>(ceil_div(nr, 256), 4096), 256, 0, st)(
       p->r_rowptr, p->r_col, p->r_w, nr, K, p->r_ell16);
@@ -855,8 +922,9 @@ static int sssp16_smem(int L, int cap, int db) { return db * L + 4 * cap + 12 * 
 
 template <int NTS, int K, typename DistT, typename OutT>
 static ear_status_t sssp16_launch(ear_plan_s *p, OutT *out, int64_t ldo, int32_t L, int32_t row0, int32_t rows,
-                                  const int32_t *trows, int cap, int smem, int32_t *counter, int32_t *sat,
+                                  const int32_t *trows, int cap, int smem, int32_t *ws,
                                   unsigned long long *d_stats, cudaStream_t st) {
+  int32_t *counter = ws, *sat = ws + 1, *wm = ws + 2, *done = ws + 4;
   constexpr int J = 2;   // two 32-vertex tasks per warp when the frontier is wide (their ELL loads overlap)
   auto kern = k_sssp16<NTS, K, J, DistT, OutT>;
   EAR_CUDA_TRY(smem_attr((const void *)kern, smem));
@@ -866,8 +934,15 @@ static ear_status_t sssp16_launch(ear_plan_s *p, OutT *out, int64_t ldo, int32_t
   int s = prof_begin(PK_SSSP, st);
   uint32_t delta = p->r_delta;
   if (const char *e = getenv("EAR_SSSP_DELTA")) delta = atoi(e) > 0 ? (uint32_t)atoi(e) : 0xFFFFFFFFu;   // lab knob
+  // row reuse (D symmetric): the single-GPU solve of every row in order -- sources 0.. with row li = source li
+  static const bool reuse_off = [] {
+    const char *e = getenv("EAR_SSSP_REUSE");   // 0: every source searches the whole graph (A/B)
+    return e && atoi(e) == 0;
+  }();
+  const uint16_t *mx = (!reuse_off && row0 == 0 && !trows) ? p->r_maxnb : nullptr;
   EAR_LAUNCH(kern, (unsigned)grid, NTS, smem, st)(reinterpret_cast<const uint4 *>(p->r_ell16), p->n_reduced, L, out,
-                                                  ldo, row0, rows, trows, cap, delta, counter, sat, d_stats);
+                                                  ldo, row0, rows, trows, cap, delta, counter, sat, mx, done, wm,
+                                                  d_stats);
   // algorithmic work: one relaxation per arc per (real) source -- Dijkstra's count; padding sources are free
   const int64_t real = trows ? rows : std::max<int64_t>(0, std::min<int64_t>(rows, (int64_t)p->n_reduced - row0));
   prof_end(s, st, (double)real * (double)p->n_rarcs);
@@ -885,13 +960,13 @@ static ear_status_t sssp16_launch(ear_plan_s *p, OutT *out, int64_t ldo, int32_t
 
 template <int NTS, typename DistT, typename OutT>
 static ear_status_t sssp16_dispatch(ear_plan_s *p, OutT *out, int64_t ldo, int32_t L, int32_t row0, int32_t rows,
-                                    const int32_t *trows, int cap, int smem, int32_t *counter, int32_t *sat,
+                                    const int32_t *trows, int cap, int smem, int32_t *ws,
                                     unsigned long long *d_stats, cudaStream_t st) {
   switch (p->r_k16) {
-    case 4: return sssp16_launch<NTS, 4, DistT, OutT>(p, out, ldo, L, row0, rows, trows, cap, smem, counter, sat, d_stats, st);
-    case 8: return sssp16_launch<NTS, 8, DistT, OutT>(p, out, ldo, L, row0, rows, trows, cap, smem, counter, sat, d_stats, st);
-    case 12: return sssp16_launch<NTS, 12, DistT, OutT>(p, out, ldo, L, row0, rows, trows, cap, smem, counter, sat, d_stats, st);
-    default: return sssp16_launch<NTS, 16, DistT, OutT>(p, out, ldo, L, row0, rows, trows, cap, smem, counter, sat, d_stats, st);
+    case 4: return sssp16_launch<NTS, 4, DistT, OutT>(p, out, ldo, L, row0, rows, trows, cap, smem, ws, d_stats, st);
+    case 8: return sssp16_launch<NTS, 8, DistT, OutT>(p, out, ldo, L, row0, rows, trows, cap, smem, ws, d_stats, st);
+    case 12: return sssp16_launch<NTS, 12, DistT, OutT>(p, out, ldo, L, row0, rows, trows, cap, smem, ws, d_stats, st);
+    default: return sssp16_launch<NTS, 16, DistT, OutT>(p, out, ldo, L, row0, rows, trows, cap, smem, ws, d_stats, st);
   }
 }
 
@@ -934,9 +1009,10 @@ static ear_status_t sssp16_rows(ear_plan_s *p, OutT *out, int64_t ldo, int32_t L
   if (const char *e = getenv("EAR_SSSP16_CAP")) cap = std::max(16, std::min(cap, atoi(e) & ~7));   // test knob: overflow
   const int smem = sssp16_smem(L, cap, db);
   if (rows <= 0) { *applied = true; return EAR_OK; }
-  int32_t *ws = nullptr;
-  EAR_CUDA_TRY(cudaMallocAsync((void **)&ws, 8, st));
-  EAR_CUDA_TRY(dev_memset(ws, 0, 8, st));
+  int32_t *ws = nullptr;   // counter, saturation flag, watermark, -, one done flag per row
+  const size_t wsb = sizeof(int32_t) * (4 + (size_t)rows);
+  EAR_CUDA_TRY(cudaMallocAsync((void **)&ws, wsb, st));
+  EAR_CUDA_TRY(dev_memset(ws, 0, wsb, st));
   static unsigned long long *d_stats = nullptr;
   static const bool want_stats = getenv("EAR_SSSP_STATS") != nullptr;
   if (want_stats && !d_stats) EAR_CUDA_TRY(cudaMalloc((void **)&d_stats, 16));
@@ -944,9 +1020,9 @@ static ear_status_t sssp16_rows(ear_plan_s *p, OutT *out, int64_t ldo, int32_t L
   unsigned long long *stt = want_stats ? d_stats : nullptr;
   ear_status_t s = EAR_OK;
   if (db == 4) {
-    s = sssp16_dispatch<SSSP16_NT, uint32_t>(p, out, ldo, L, row0, rows, trows, cap, smem, ws, ws + 1, stt, st);
+    s = sssp16_dispatch<SSSP16_NT, uint32_t>(p, out, ldo, L, row0, rows, trows, cap, smem, ws, stt, st);
   } else {
-    s = sssp16_dispatch<SSSP16_NT, uint16_t>(p, out, ldo, L, row0, rows, trows, cap, smem, ws, ws + 1, stt, st);
+    s = sssp16_dispatch<SSSP16_NT, uint16_t>(p, out, ldo, L, row0, rows, trows, cap, smem, ws, stt, st);
   }
   int32_t h_sat = 1;
   if (s == EAR_OK) {
