@@ -749,6 +749,30 @@ static ear_status_t reduce_solve(const ear_plan_s *p, int32_t n, int64_t m, cons
   const int64_t unit = (int64_t)TILE * (comm ? comm->nranks : 1);
   const bool worth = s == EAR_OK && (by_sssp ? depth == 0 || q->n_reduced < n
                                              : round_up(std::max<int64_t>(q->n_reduced, 1), unit) < round_up(n, unit));
+  if (s == EAR_OK && by_sssp && !comm && depth == 0 && (int64_t)q->n_reduced * 10 > (int64_t)n * 9) {
+    // the contraction removes < 10 % of the piece: its Phase III pass (a gather per entry of the piece
+    // matrix; cfg4's root piece: 4.2 ms for 405 vertices removed) costs more than the SSSP work it saves
+    // (~n^2 scaling, 1.8 ms).  Run the SSSP on the piece itself instead -- every vertex a terminal, so
+    // the plan's ids are the piece's own -- with the rows written straight into M.
+    cudaStreamSynchronize(st);
+    plan_free(q);
+    delete q;
+    q = new ear_plan_s;
+    q->device = p->device;
+    s = decompose(n, m, u, v, w, EAR_FLAG_NO_CONTRACT | (p->flags & EAR_FLAG_FW32), st, q);
+    const int32_t Lp = (int32_t)round_up(std::max<int64_t>(n, 1), (int64_t)TILE);
+    if (s == EAR_OK && ld >= Lp) s = sssp_rows(q, M, ld, Lp, 0, n, nullptr, st);
+    else if (s == EAR_OK) s = EAR_EUNSUPPORTED;   // (pool matrices are padded to whole tiles)
+    cudaStreamSynchronize(st);
+    plan_free(q);
+    delete q;
+    if (s == EAR_OK) {
+      *done = true;
+      *levels = depth;
+      *n_last = n;
+    }
+    return s;
+  }
   if (!worth) {
     cudaStreamSynchronize(st);
     plan_free(q);

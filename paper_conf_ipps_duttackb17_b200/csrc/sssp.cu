@@ -431,7 +431,8 @@ __global__ void __launch_bounds__(NTS, 3) k_sssp16(const uint4 *__restrict__ ell
   uint32_t *Mb = reinterpret_cast<uint32_t *>(dist + L);                     // [2][W]
   uint32_t *F = Mb + 2 * W;                                                  // [W] the far pile
   uint16_t *Lb = reinterpret_cast<uint16_t *>(F + W);                        // [2][NW][S]
-  __shared__ int scnt[3][NW], ovf[3], s_item, s_sat;
+  __shared__ __align__(16) int scnt[3][NW];
+  __shared__ int ovf[3], s_item, s_sat;
   __shared__ uint32_t s_min[NW];
   __shared__ int s_red[NW], s_k;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -522,12 +523,33 @@ __global__ void __launch_bounds__(NTS, 3) k_sssp16(const uint4 *__restrict__ ell
           const uint32_t u = a & 0xFFFFu;
           if (u == 0xFFFFu) return false;
           const uint32_t nd = dv + (a >> 16);
-          const uint32_t cur = dist[u];
-          if (nd >= 0xFFFFu) {   // not representable: harmless unless u stays unreached
-            if (cur == DINF) s_sat = 1;
-            return false;
+          uint32_t cur;
+          if constexpr (sizeof(DistT) == 2) {
+            // the 32-bit word holding d(u): one LDS, and a CAS on the word (the compiler's 16-bit CAS
+            // emulation costs ~22 instructions)
+            uint32_t *wp = reinterpret_cast<uint32_t *>(dist) + (u >> 1);
+            const uint32_t sh = (u & 1u) << 4;
+            uint32_t w = *wp;
+            cur = (w >> sh) & 0xFFFFu;
+            if (nd >= 0xFFFFu) {   // not representable: harmless unless u stays unreached
+              if (cur == DINF) s_sat = 1;
+              return false;
+            }
+            for (;;) {
+              if (nd >= cur) return false;
+              const uint32_t prev = atomicCAS(wp, w, w ^ ((cur ^ nd) << sh));
+              if (prev == w) break;
+              w = prev;
+              cur = (w >> sh) & 0xFFFFu;
+            }
+          } else {
+            cur = dist[u];
+            if (nd >= 0xFFFFu) {
+              if (cur == DINF) s_sat = 1;
+              return false;
+            }
+            if (nd >= cur || !sssp_lower(dist + u, nd, cur)) return false;
           }
-          if (nd >= cur || !sssp_lower(dist + u, nd, cur)) return false;
           if (stats) ++my_relax;
           const uint32_t bit = 1u << (u & 31);
           if (nd >= thr) {   // far: waits for the threshold
@@ -539,8 +561,16 @@ __global__ void __launch_bounds__(NTS, 3) k_sssp16(const uint4 *__restrict__ ell
         if (!scan) {
           int pre[NW + 1];
           pre[0] = 0;
+          {
+            int c[NW];
 #pragma unroll
-          for (int w = 0; w < NW; ++w) pre[w + 1] = pre[w] + min(scnt[r % 3][w], S);
+            for (int q = 0; q < NW / 4; ++q) {
+              const int4 c4 = reinterpret_cast<const int4 *>(scnt[r % 3])[q];
+              c[4 * q] = c4.x; c[4 * q + 1] = c4.y; c[4 * q + 2] = c4.z; c[4 * q + 3] = c4.w;
+            }
+#pragma unroll
+            for (int w = 0; w < NW; ++w) pre[w + 1] = pre[w] + min(c[w], S);
+          }
           const int n = pre[NW], ntask = (n + 31) >> 5;
           for (int w = w0; w < w1; ++w) Mc[w] = 0u;   // nobody sets Mc this round
           int wc = 0;                                 // warp-uniform append offset
@@ -612,7 +642,10 @@ __global__ void __launch_bounds__(NTS, 3) k_sssp16(const uint4 *__restrict__ ell
         ++my_rounds;
         int more = ovf[(r + 1) % 3];
 #pragma unroll
-        for (int w = 0; w < NW; ++w) more |= scnt[(r + 1) % 3][w];
+        for (int q = 0; q < NW / 4; ++q) {
+          const int4 c4 = reinterpret_cast<const int4 *>(scnt[(r + 1) % 3])[q];
+          more |= c4.x | c4.y | c4.z | c4.w;
+        }
         if (more) continue;
         // the near pile is empty: raise the threshold to (smallest live far distance) + delta and list
         // the far vertices below it for round r+1.  A far entry already below the old threshold is stale
