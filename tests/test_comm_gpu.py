@@ -24,7 +24,8 @@ def test_one_rank_comm_path():
     try:
         for g in [gg.config("cfg1"), gg.corner_cases(12, n_target=500), decorated_grid(24, 0.3, 0)]:
             ref = oracle.apsp(g.n, g.src, g.dst, g.w)
-            for flags in (0, ea.FLAG_SSSP, ea.FLAG_BCC, ea.FLAG_FW32, ea.FLAG_BCC | ea.FLAG_FW32):
+            for flags in (0, ea.FLAG_SSSP, ea.FLAG_BCC, ea.FLAG_FW32, ea.FLAG_BCC | ea.FLAG_FW32,
+                          ea.FLAG_BCC | ea.FLAG_SSSP):
                 out = ea.apsp_full(g.n, dev(g.src), dev(g.dst), dev(g.w), comm=comm, flags=flags)
                 torch.cuda.synchronize()
                 assert np.array_equal(out.cpu().numpy(), ref), f"comm path mismatch (flags={flags})"

@@ -1,7 +1,7 @@
 """Full N x N verification at the north-star sizes (S defined at P:109; SURVEY 8.c pin P4).
 
 Every entry of cfg4's matrix (100k vertices, 40 GB) in the bench's launch configuration (apsp_full,
-Phase II by biconnected pieces), and -- with EAR_VERIFY_CFG5=1 -- every entry of cfg5's (200k vertices,
+Phase II by biconnected pieces solved by per-source SSSP) and by the blocked-FW route, and -- with EAR_VERIFY_CFG5=1 -- every entry of cfg5's (200k vertices,
 160 GB: Phase II once, the expansion in row blocks) is checked by the oracle's Bellman certificate
 (oracle.certify_rows: the definition of S restated as a fixed point whose only solution is S) on the
 host's cores, streaming row blocks device -> pinned host while the previous block is being certified.
@@ -73,30 +73,40 @@ def report(summary):
     print(json.dumps(summary))
 
 
-def test_cfg4_full_matrix_certified():
+ROUTES = {"bcc_sssp": ("FLAG_BCC | FLAG_SSSP (bench default)", lambda ea: ea.FLAG_BCC | ea.FLAG_SSSP),
+          "bcc_fw": ("FLAG_BCC (pieces by the blocked FW)", lambda ea: ea.FLAG_BCC)}
+
+
+@pytest.mark.parametrize("route", list(ROUTES))
+def test_cfg4_full_matrix_certified(route):
     import paper_conf_ipps_duttackb17_b200 as ea
     g = gg.config("cfg4")
+    name, fl = ROUTES[route]
+    flags = fl(ea)
     out = torch.empty((g.n, g.n), dtype=torch.int32, device="cuda")
     src, dst, w = dev(g.src), dev(g.dst), dev(g.w)
-    ea.apsp_full(g.n, src, dst, w, out=out, flags=ea.FLAG_BCC)   # warm-up (the bench's configuration)
+    ea.apsp_full(g.n, src, dst, w, out=out, flags=flags)   # warm-up
     torch.cuda.synchronize()
     t = time.perf_counter()
-    ea.apsp_full(g.n, src, dst, w, out=out, flags=ea.FLAG_BCC)
+    ea.apsp_full(g.n, src, dst, w, out=out, flags=flags)
     torch.cuda.synchronize()
     gpu_s = time.perf_counter() - t
     s = certify_stream(g, lambda r0, r1: out[r0:r1], 5000)
-    s.update({"config": "cfg4", "n": g.n, "m": g.m, "path": "apsp_full FLAG_BCC (bench default), one call",
-              "gpu_apsp_full_s": gpu_s})
+    s.update({"config": "cfg4", "n": g.n, "m": g.m, "path": f"apsp_full {name}, one call", "gpu_apsp_full_s": gpu_s})
+    del out
+    torch.cuda.empty_cache()
     report(s)
     assert s["violations"] == 0, s
 
 
 @pytest.mark.skipif(os.environ.get("EAR_VERIFY_CFG5") != "1", reason="cfg5 full check: EAR_VERIFY_CFG5=1 (~3 min)")
-def test_cfg5_full_matrix_certified():
+@pytest.mark.parametrize("route", list(ROUTES))
+def test_cfg5_full_matrix_certified(route):
     import paper_conf_ipps_duttackb17_b200 as ea
     g = gg.config("cfg5")
+    name, fl = ROUTES[route]
     src, dst, w = dev(g.src), dev(g.dst), dev(g.w)
-    plan = ea.ear_decompose(g.n, src, dst, w, flags=ea.FLAG_BCC)
+    plan = ea.ear_decompose(g.n, src, dst, w, flags=fl(ea))
     D = ea.alloc_D(plan)
     t = time.perf_counter()
     ea.apsp_reduced(plan, D)
@@ -115,8 +125,10 @@ def test_cfg5_full_matrix_certified():
 
     s = certify_stream(g, produce, rows)
     s.update({"config": "cfg5", "n": g.n, "m": g.m, "n_reduced": plan.info().n_reduced,
-              "path": "ear_decompose FLAG_BCC + apsp_reduced once + expand_ears by 10,000-row blocks (one B200)",
+              "path": f"ear_decompose {name} + apsp_reduced once + expand_ears by 10,000-row blocks (one B200)",
               "gpu_phase2_s": phase2_s, "gpu_expand_s": t_exp[0]})
     plan.destroy()
+    del D, out
+    torch.cuda.empty_cache()
     report(s)
     assert s["violations"] == 0, s
