@@ -417,7 +417,7 @@ __device__ __forceinline__ bool sssp_lower(DistT *d, uint32_t nd, uint32_t cur) 
 }
 
 template <int NTS, int K, int J, typename DistT, typename OutT>
-__global__ void __launch_bounds__(NTS, 3) k_sssp16(const uint4 *__restrict__ ell, int32_t nr, int32_t L, OutT *out,
+__global__ void __launch_bounds__(NTS, 768 / NTS) k_sssp16(const uint4 *__restrict__ ell, int32_t nr, int32_t L, OutT *out,
                                                int64_t ldo, int32_t src0, int32_t nsrc, const int32_t *trows, int cap,
                                                uint32_t delta, int32_t *counter, int32_t *sat,
                                                const uint16_t *__restrict__ maxnb, int32_t *done, int32_t *wm,
@@ -426,11 +426,12 @@ __global__ void __launch_bounds__(NTS, 3) k_sssp16(const uint4 *__restrict__ ell
   constexpr uint32_t DINF = sizeof(DistT) == 2 ? 0xFFFFu : 0xFFFFFFFFu;
   extern __shared__ __align__(16) uint32_t smw[];
   const int W = (L + 31) >> 5;
+  const int WS = (W + 3) & ~3;                                               // bitmap stride (16-byte rows)
   const int S = cap / NW;                                                    // segment length
   DistT *dist = reinterpret_cast<DistT *>(smw);                              // [L], L % 8 == 0
-  uint32_t *Mb = reinterpret_cast<uint32_t *>(dist + L);                     // [2][W]
-  uint32_t *F = Mb + 2 * W;                                                  // [W] the far pile
-  uint16_t *Lb = reinterpret_cast<uint16_t *>(F + W);                        // [2][NW][S]
+  uint32_t *Mb = reinterpret_cast<uint32_t *>(dist + L);                     // [2][WS]
+  uint32_t *F = Mb + 2 * WS;                                                 // [WS] the far pile
+  uint16_t *Lb = reinterpret_cast<uint16_t *>(F + WS);                       // [2][NW][S]
   __shared__ __align__(16) int scnt[3][NW];
   __shared__ int ovf[3], s_item, s_sat;
   __shared__ uint32_t s_min[NW];
@@ -472,7 +473,7 @@ __global__ void __launch_bounds__(NTS, 3) k_sssp16(const uint4 *__restrict__ ell
     }
     for (int i = tid; i < L * (int)sizeof(DistT) / 16; i += NTS)
       reinterpret_cast<uint4 *>(dist)[i] = make_uint4(~0u, ~0u, ~0u, ~0u);
-    for (int w = tid; w < 2 * W; w += NTS) Mb[w] = 0u;   // both list bitmaps
+    for (int w = tid; w < 2 * WS; w += NTS) Mb[w] = 0u;   // both list bitmaps
     if (tid < 3 * NW) (&scnt[0][0])[tid] = 0;
     if (tid < 3) ovf[tid] = 0;
     if (tid == 0) s_sat = 0;
@@ -509,15 +510,17 @@ __global__ void __launch_bounds__(NTS, 3) k_sssp16(const uint4 *__restrict__ ell
     __syncthreads();
     if (src < nr) {
       uint32_t thr = 0;   // near-far: only vertices below thr are expanded (uniform)
+      int c0 = 0, c1 = 1, c2 = 2, par = 0;   // count slots of rounds r, r+1, r+2 (r % 3 ...) and r & 1
       for (int r = 0;; ++r) {
-        const uint16_t *Lc = Lb + (r & 1) * (NW * S);
-        uint16_t *Ln = Lb + ((r + 1) & 1) * (NW * S) + warp * S;   // this warp's segment
-        uint32_t *Mc = Mb + (r & 1) * W, *Mn = Mb + ((r + 1) & 1) * W;
-        const bool scan = ovf[r % 3] != 0;
-        int *ncnt = &scnt[(r + 1) % 3][warp];
-        int *novf = &ovf[(r + 1) % 3];
-        if (tid < NW) scnt[(r + 2) % 3][tid] = 0;
-        if (tid == 0) ovf[(r + 2) % 3] = 0;
+        const uint16_t *Lc = Lb + par * (NW * S);
+        uint16_t *Ln = Lb + (par ^ 1) * (NW * S) + warp * S;   // this warp's segment
+        uint32_t *Mc = Mb + par * WS, *Mn = Mb + (par ^ 1) * WS;
+        const bool scan = ovf[c0] != 0;
+        int *ncnt = &scnt[c1][warp];
+        int *novf = &ovf[c1];
+        if (tid < NW) scnt[c2][tid] = 0;
+        if (tid == 0) ovf[c2] = 0;
+        int wc = 0;   // warp-uniform append offset into this warp's segment
         // relax arc a from a vertex at distance dv; true when u is new on round r+1's list
         auto relax = [&](uint32_t dv, uint32_t a) -> bool {
           const uint32_t u = a & 0xFFFFu;
@@ -559,34 +562,66 @@ __global__ void __launch_bounds__(NTS, 3) k_sssp16(const uint4 *__restrict__ ell
           return !(atomicOr(&Mn[u >> 5], bit) & bit);
         };
         if (!scan) {
+          int c[NW];
+#pragma unroll
+          for (int q = 0; q < NW / 4; ++q) {
+            const int4 c4 = reinterpret_cast<const int4 *>(scnt[c0])[q];
+            c[4 * q] = min(c4.x, S); c[4 * q + 1] = min(c4.y, S); c[4 * q + 2] = min(c4.z, S); c[4 * q + 3] = min(c4.w, S);
+          }
+          int n = 0;
+#pragma unroll
+          for (int w = 0; w < NW; ++w) n += c[w];
+          const int ntask = (n + 31) >> 5;
+          for (int q = tid; q < WS / 4; q += NTS)   // nobody sets Mc this round
+            reinterpret_cast<uint4 *>(Mc)[q] = make_uint4(0u, 0u, 0u, 0u);
+          // a narrow frontier leaves warps idle: then f warps share each task, warp g taking the ELL
+          // groups g and g + f (4 arcs each) -- the slot chain a task warp runs serially gets f times shorter
+          int f = 1;
+          if (K / 4 > 1)
+            while (2 * f <= K / 4 && ntask * 2 * f <= NW) f *= 2;
           int pre[NW + 1];
           pre[0] = 0;
-          {
-            int c[NW];
+          if (warp < ntask * f) {   // (only warps holding a task look entries up)
 #pragma unroll
-            for (int q = 0; q < NW / 4; ++q) {
-              const int4 c4 = reinterpret_cast<const int4 *>(scnt[r % 3])[q];
-              c[4 * q] = c4.x; c[4 * q + 1] = c4.y; c[4 * q + 2] = c4.z; c[4 * q + 3] = c4.w;
-            }
-#pragma unroll
-            for (int w = 0; w < NW; ++w) pre[w + 1] = pre[w] + min(c[w], S);
+            for (int w = 0; w < NW; ++w) pre[w + 1] = pre[w] + c[w];
           }
-          const int n = pre[NW], ntask = (n + 31) >> 5;
-          for (int w = w0; w < w1; ++w) Mc[w] = 0u;   // nobody sets Mc this round
-          int wc = 0;                                 // warp-uniform append offset
+          auto entry = [&](int i) -> int {
+            int sg = 0;
+#pragma unroll
+            for (int w = 1; w < NW; ++w) sg += i >= pre[w];
+            return Lc[sg * S + i - pre[sg]];
+          };
+          if (f > 1) {
+            if (warp < ntask * f) {   // warp-uniform
+              const int t = warp % ntask, g = warp / ntask, i = t * 32 + lane;
+              const int v = i < n ? entry(i) : -1;
+              const uint4 *row = ell + (int64_t)max(v, 0) * (K / 4);
+              const uint4 pad = make_uint4(~0u, ~0u, ~0u, ~0u);
+              const uint4 e0 = v >= 0 ? __ldg(row + g) : pad;
+              const uint4 e1 = (v >= 0 && g + f < K / 4) ? __ldg(row + g + f) : pad;
+              const uint32_t dv = v >= 0 ? (uint32_t)dist[v] : 0u;
+#pragma unroll
+              for (int k = 0; k < 8; ++k) {
+                const uint4 q = k < 4 ? e0 : e1;
+                const uint32_t a = (k & 3) == 0 ? q.x : (k & 3) == 1 ? q.y : (k & 3) == 2 ? q.z : q.w;
+                if (!__any_sync(0xFFFFFFFFu, (a & 0xFFFFu) != 0xFFFFu)) break;   // padding from here on
+                const bool push = relax(dv, a);
+                const unsigned bal = __ballot_sync(0xFFFFFFFFu, push);
+                if (push) {
+                  const int idx = wc + __popc(bal & lt);
+                  if (idx < S) Ln[idx] = (uint16_t)(a & 0xFFFFu);
+                }
+                wc += __popc(bal);
+              }
+            }
+          } else
           for (int t0 = warp; t0 < ntask; t0 += J * NW) {   // warp-uniform: the ballots see all lanes
             int vv[J];
             uint4 e[J][K / 4];
 #pragma unroll
             for (int j = 0; j < J; ++j) {
               const int i = (t0 + j * NW) * 32 + lane;
-              vv[j] = -1;
-              if (i < n) {
-                int sg = 0;
-#pragma unroll
-                for (int w = 1; w < NW; ++w) sg += i >= pre[w];
-                vv[j] = Lc[sg * S + i - pre[sg]];
-              }
+              vv[j] = i < n ? entry(i) : -1;
               const uint4 *row = ell + (int64_t)max(vv[j], 0) * (K / 4);
 #pragma unroll
               for (int k = 0; k < K / 4; ++k) e[j][k] = vv[j] >= 0 ? __ldg(row + k) : make_uint4(~0u, ~0u, ~0u, ~0u);
@@ -640,11 +675,16 @@ __global__ void __launch_bounds__(NTS, 3) k_sssp16(const uint4 *__restrict__ ell
         }
         __syncthreads();
         ++my_rounds;
-        int more = ovf[(r + 1) % 3];
+        int more = ovf[c1];
 #pragma unroll
         for (int q = 0; q < NW / 4; ++q) {
-          const int4 c4 = reinterpret_cast<const int4 *>(scnt[(r + 1) % 3])[q];
+          const int4 c4 = reinterpret_cast<const int4 *>(scnt[c1])[q];
           more |= c4.x | c4.y | c4.z | c4.w;
+        }
+        {   // rotate the slots for round r+1
+          const int t = c0;
+          c0 = c1; c1 = c2; c2 = t;
+          par ^= 1;
         }
         if (more) continue;
         // the near pile is empty: raise the threshold to (smallest live far distance) + delta and list
@@ -671,8 +711,8 @@ __global__ void __launch_bounds__(NTS, 3) k_sssp16(const uint4 *__restrict__ ell
         const uint32_t told = thr;
         thr = mn + delta;
         {
-          uint32_t *Mn = Mb + ((r + 1) & 1) * W;   // round r+1's list bitmap (owned words: plain stores)
-          uint16_t *Ln = Lb + ((r + 1) & 1) * (NW * S) + warp * S;
+          uint32_t *Mn = Mb + par * WS;   // round r+1's list bitmap (owned words: plain stores)
+          uint16_t *Ln = Lb + par * (NW * S) + warp * S;
           int wc = 0;
           for (int wb = warp * 32 * wpt; wb < W; wb += NTS * wpt) {   // warp-uniform over the owned words
             for (int q = 0; q < wpt; ++q) {
@@ -702,8 +742,8 @@ __global__ void __launch_bounds__(NTS, 3) k_sssp16(const uint4 *__restrict__ ell
             }
           }
           if (lane == 0) {
-            scnt[(r + 1) % 3][warp] = wc;
-            if (wc > S) ovf[(r + 1) % 3] = 1;
+            scnt[c0][warp] = wc;
+            if (wc > S) ovf[c0] = 1;
           }
         }
         __syncthreads();
@@ -951,7 +991,7 @@ static ear_status_t ell16_prepare(ear_plan_s *p, cudaStream_t st) {
 constexpr int SSSP16_NT = 256;
 constexpr int SSSP16_MAX_CTAS = 2048 / SSSP16_NT;
 // shared memory of one source: the row (L entries of db bytes), two lists (cap u16 each), three bitmaps
-static int sssp16_smem(int L, int cap, int db) { return db * L + 4 * cap + 12 * ((L + 31) / 32); }
+static int sssp16_smem(int L, int cap, int db) { return db * L + 4 * cap + 12 * (((L + 31) / 32 + 3) & ~3); }
 
 template <int NTS, int K, typename DistT, typename OutT>
 static ear_status_t sssp16_launch(ear_plan_s *p, OutT *out, int64_t ldo, int32_t L, int32_t row0, int32_t rows,
@@ -1052,7 +1092,14 @@ static ear_status_t sssp16_rows(ear_plan_s *p, OutT *out, int64_t ldo, int32_t L
   if (want_stats) EAR_CUDA_TRY(dev_memset(d_stats, 0, 16, st));
   unsigned long long *stt = want_stats ? d_stats : nullptr;
   ear_status_t s = EAR_OK;
-  if (db == 4) {
+  static const int nt_lab = [] {
+    const char *e = getenv("EAR_SSSP16_NT");   // lab knob: 128 threads per source
+    return e ? atoi(e) : 0;
+  }();
+  if (nt_lab == 128) {
+    s = db == 4 ? sssp16_dispatch<128, uint32_t>(p, out, ldo, L, row0, rows, trows, cap, smem, ws, stt, st)
+                : sssp16_dispatch<128, uint16_t>(p, out, ldo, L, row0, rows, trows, cap, smem, ws, stt, st);
+  } else if (db == 4) {
     s = sssp16_dispatch<SSSP16_NT, uint32_t>(p, out, ldo, L, row0, rows, trows, cap, smem, ws, stt, st);
   } else {
     s = sssp16_dispatch<SSSP16_NT, uint16_t>(p, out, ldo, L, row0, rows, trows, cap, smem, ws, stt, st);
