@@ -402,6 +402,27 @@ __global__ void __launch_bounds__(NTS) k_sssp_list(const int2 *__restrict__ ell,
 // vertex marks the source, and a marked source whose row keeps an unreached vertex raises *sat: the
 // caller then falls back to int32 (every shortest path's prefixes are below the final distance, so a
 // row without unreached vertices is exact).
+// shared-memory accesses by 32-bit shared-window address (computed once per kernel): the generic-pointer
+// atomics re-derived the window base (S2R + 3 ALU) in every relaxation
+__device__ __forceinline__ uint32_t lds_u32(uint32_t a) {
+  uint32_t v;
+  asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(a) : "memory");
+  return v;
+}
+__device__ __forceinline__ uint32_t atoms_cas(uint32_t a, uint32_t cmp, uint32_t val) {
+  uint32_t o;
+  asm volatile("atom.shared.cas.b32 %0, [%1], %2, %3;" : "=r"(o) : "r"(a), "r"(cmp), "r"(val) : "memory");
+  return o;
+}
+__device__ __forceinline__ uint32_t atoms_or(uint32_t a, uint32_t val) {
+  uint32_t o;
+  asm volatile("atom.shared.or.b32 %0, [%1], %2;" : "=r"(o) : "r"(a), "r"(val) : "memory");
+  return o;
+}
+__device__ __forceinline__ void reds_or(uint32_t a, uint32_t val) {
+  asm volatile("red.shared.or.b32 [%0], %1;" ::"r"(a), "r"(val) : "memory");
+}
+
 template <typename DistT>
 __device__ __forceinline__ bool sssp_lower(DistT *d, uint32_t nd, uint32_t cur) {
   if constexpr (sizeof(DistT) == 4) {
@@ -432,6 +453,8 @@ __global__ void __launch_bounds__(NTS, 768 / NTS) k_sssp16(const uint4 *__restri
   uint32_t *Mb = reinterpret_cast<uint32_t *>(dist + L);                     // [2][WS]
   uint32_t *F = Mb + 2 * WS;                                                 // [WS] the far pile
   uint16_t *Lb = reinterpret_cast<uint16_t *>(F + WS);                       // [2][NW][S]
+  const uint32_t dist_s = (uint32_t)__cvta_generic_to_shared(dist);
+  const uint32_t F_s = (uint32_t)__cvta_generic_to_shared(F);
   __shared__ __align__(16) int scnt[3][NW];
   __shared__ int ovf[3], s_item, s_sat;
   __shared__ uint32_t s_min[NW];
@@ -515,6 +538,7 @@ __global__ void __launch_bounds__(NTS, 768 / NTS) k_sssp16(const uint4 *__restri
         const uint16_t *Lc = Lb + par * (NW * S);
         uint16_t *Ln = Lb + (par ^ 1) * (NW * S) + warp * S;   // this warp's segment
         uint32_t *Mc = Mb + par * WS, *Mn = Mb + (par ^ 1) * WS;
+        const uint32_t Mn_s = (uint32_t)__cvta_generic_to_shared(Mn);
         const bool scan = ovf[c0] != 0;
         int *ncnt = &scnt[c1][warp];
         int *novf = &ovf[c1];
@@ -530,9 +554,9 @@ __global__ void __launch_bounds__(NTS, 768 / NTS) k_sssp16(const uint4 *__restri
           if constexpr (sizeof(DistT) == 2) {
             // the 32-bit word holding d(u): one LDS, and a CAS on the word (the compiler's 16-bit CAS
             // emulation costs ~22 instructions)
-            uint32_t *wp = reinterpret_cast<uint32_t *>(dist) + (u >> 1);
+            const uint32_t wa = dist_s + ((u << 1) & ~3u);
             const uint32_t sh = (u & 1u) << 4;
-            uint32_t w = *wp;
+            uint32_t w = lds_u32(wa);
             cur = (w >> sh) & 0xFFFFu;
             if (nd >= 0xFFFFu) {   // not representable: harmless unless u stays unreached
               if (cur == DINF) s_sat = 1;
@@ -540,7 +564,7 @@ __global__ void __launch_bounds__(NTS, 768 / NTS) k_sssp16(const uint4 *__restri
             }
             for (;;) {
               if (nd >= cur) return false;
-              const uint32_t prev = atomicCAS(wp, w, w ^ ((cur ^ nd) << sh));
+              const uint32_t prev = atoms_cas(wa, w, w ^ ((cur ^ nd) << sh));
               if (prev == w) break;
               w = prev;
               cur = (w >> sh) & 0xFFFFu;
@@ -556,10 +580,10 @@ __global__ void __launch_bounds__(NTS, 768 / NTS) k_sssp16(const uint4 *__restri
           if (stats) ++my_relax;
           const uint32_t bit = 1u << (u & 31);
           if (nd >= thr) {   // far: waits for the threshold
-            atomicOr(&F[u >> 5], bit);
+            reds_or(F_s + ((u >> 5) << 2), bit);
             return false;
           }
-          return !(atomicOr(&Mn[u >> 5], bit) & bit);
+          return !(atoms_or(Mn_s + ((u >> 5) << 2), bit) & bit);
         };
         if (!scan) {
           int c[NW];
