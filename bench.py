@@ -272,9 +272,14 @@ def run_ours(args, rank, world, local_rank):
     plan.destroy()
     stream = torch.cuda.current_stream(dev)
 
-    flags = {"fw": 0, "sssp": ea.FLAG_SSSP, "bcc": ea.FLAG_BCC, "bcc_sssp": ea.FLAG_BCC | ea.FLAG_SSSP}[args.phase2] \
+    flags = {"fw": 0, "sssp": ea.FLAG_SSSP, "bcc": ea.FLAG_BCC, "bcc_sssp": ea.FLAG_BCC | ea.FLAG_SSSP,
+             "part": ea.FLAG_PART | ea.FLAG_BCC | ea.FLAG_SSSP}[args.phase2] \
         | (ea.FLAG_FW32 if args.fw32 else 0)
-    bcc = None
+    bcc = part = None
+    if args.phase2 == "part":
+        pp = ea.ear_decompose(g.n, src, dst, w, flags=flags)
+        part = pp.part_info()
+        pp.destroy()
     if args.phase2 in ("bcc", "bcc_sssp"):
         pb = ea.ear_decompose(g.n, src, dst, w, flags=flags)
         if world == 1 and not args.no_alt:   # one untimed Phase II: the re-reduction counts of a solve
@@ -388,7 +393,23 @@ def run_ours(args, rank, world, local_rank):
                                   "DESIGN.md 6b)"}
         if clocks.get("sm_mhz"):
             roofline["frac_at_run_clock"] = ach / (SM_COUNT * 32 * clocks["sm_mhz"] * 1e6 / 1e9)
-    phases = {"decompose": prof["decompose_ms"] / K, "fw": fw_ms / K, "sssp": prof["sssp_ms"] / K, "fw_phase1": prof["fw_phase1_ms"] / K,
+    if args.phase2 == "part" and prof["part_mp_ms"] > 0:   # the region products (ALU, packed u16x2)
+        pm_ms = prof["part_mp_ms"]
+        n_pm = max(prof["part_mp_launches"], 1)
+        ach = prof["part_minplus"] / (pm_ms / 1e3) / 1e12
+        lanes = 2 * ALU_LANES_PER_SM
+        peak_alu = SM_COUNT * lanes * sm_max * 1e6 / 1e12
+        roofline = {"bound": "alu", "kernel": "k_region_mp (Phase II by regions: min-plus products through the "
+                                              "region boundaries, packed u16x2)",
+                    "achieved": ach, "peak": peak_alu, "unit": "Tminplus/s", "frac": ach / peak_alu,
+                    "traffic": ncu_traffic("k_region_mp", args.config), "avg_launch_ms": pm_ms / n_pm,
+                    "minplus_per_launch": prof["part_minplus"] / n_pm,
+                    "peak_basis": f"{SM_COUNT} SMs x {lanes} min-plus/clk/SM (64 VIADDMNMX.U16x2, two lanes each) "
+                                  f"x {sm_max:.0f} MHz (sm_max_mhz of MEASURED_PEAKS.json; issue rate from "
+                                  "microbench/minplus_peak.cu)"}
+        if clocks.get("sm_mhz"):
+            roofline["frac_at_run_clock"] = ach / (SM_COUNT * lanes * clocks["sm_mhz"] * 1e6 / 1e12)
+    phases = {"decompose": prof["decompose_ms"] / K, "part": prof["part_ms"] / K, "part_mp": prof["part_mp_ms"] / K, "fw": fw_ms / K, "sssp": prof["sssp_ms"] / K, "fw_phase1": prof["fw_phase1_ms"] / K,
               "fw_phase2": prof["fw_phase2_ms"] / K, "fw_phase3": p3_ms / K, "comm": prof["comm_ms"] / K,
               "expand": ex_ms / K, "same_chain": prof["same_chain_ms"] / K,
               "bcc_pieces": prof["bcc_pieces_ms"] / K, "compose": prof["compose_ms"] / K,
@@ -404,7 +425,8 @@ def run_ours(args, rank, world, local_rank):
     alt = None
     if world == 1 and not args.no_alt:
         alt = {"note": "Phase II only (D of G^r), one timed call after a warm-up call; --phase2 X times the full step"}
-        for name, fl in (("fw", 0), ("sssp", ea.FLAG_SSSP), ("bcc", ea.FLAG_BCC), ("bcc_sssp", ea.FLAG_BCC | ea.FLAG_SSSP)):
+        for name, fl in (("fw", 0), ("sssp", ea.FLAG_SSSP), ("bcc", ea.FLAG_BCC), ("bcc_sssp", ea.FLAG_BCC | ea.FLAG_SSSP),
+                         ("part", ea.FLAG_PART)):
             if name == args.phase2:
                 continue
             p2 = ea.ear_decompose(g.n, src, dst, w, flags=fl)
@@ -513,7 +535,7 @@ def run_ours(args, rank, world, local_rank):
                            "n_chains": info.n_chains, "max_chain_len": info.max_chain_len,
                            "degree2_frac": stats["deg2_frac"], "seed": args.seed, "rows_per_rank": rows,
                            "parallelism": f"row-block x{world}" if world > 1 else "single GPU",
-                           "phase2": args.phase2, "bcc": bcc,
+                           "phase2": args.phase2, "bcc": bcc, "part": part,
                            "l2": "inputs larger than L2 (D %.1f GB, output %.1f GB per step)" % (
                                4.0 * info.n_reduced_padded ** 2 / 1e9, 4.0 * g.n * g.n / 1e9)},
                 "roofline": roofline, "roofline_expand": roofline_expand,
@@ -538,7 +560,7 @@ def main():
     ap.add_argument("--config", default="cfg4")
     ap.add_argument("--seed", type=int, default=0)
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
-    ap.add_argument("--phase2", choices=["bcc_sssp", "bcc", "fw", "sssp"], default="bcc_sssp",
+    ap.add_argument("--phase2", choices=["part", "bcc_sssp", "bcc", "fw", "sssp"], default="bcc_sssp",
                     help="Phase II: the biconnected pieces of G^r (paper sec. 2.2) each reduced again and solved by "
                          "per-source SSSP (the paper's own Phase II, P:101; default), the same pieces by blocked FW, "
                          "blocked FW on all of G^r, or per-source SSSP on all of G^r")

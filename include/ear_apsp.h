@@ -59,6 +59,15 @@ enum {
                                bit for bit.  With EAR_FLAG_SSSP too, every big piece is reduced again
                                 and its reduced graph solved by the per-source SSSP instead of
                                the FW (the bench's route: O(n m) work per piece instead of O(n^3)). */
+  EAR_FLAG_PART = 16,       /* Phase II by regions (reading C24): G^r cut into connected
+                               regions of <= 256 vertices (Voronoi cells of a multi-source BFS), the
+                               distances inside every region by one CTA each, the distances between
+                               region boundaries by a blocked FW on the boundary graph, and every row of D
+                               by two min-plus products with a region boundary as the inner dimension --
+                               sec. 2.2's composition through articulation points with
+                               boundary sets as the separators.  Same D bit for bit; applies when the
+                               distances fit u16 sums (else the SSSP / FW route of the other flags runs).
+                               The bench's route. */
   EAR_FLAG_FW32 = 8         /* single-GPU FW: skip the packed 16-bit attempt and run int32 throughout.
                                By default the FW first runs on a copy of D capped at 0x7FFF with two
                                min-plus per VIADDMNMX.U16x2 (exact for every distance < 0x7FFF, see
@@ -193,6 +202,20 @@ typedef struct {
                                 piece is reduced again while that removes >= 1 % of its vertices) */
 } ear_bcc_info_t;
 ear_status_t ear_bcc_info(ear_plan_t plan, ear_bcc_info_t *info);
+
+/* Region partition used by EAR_FLAG_PART (built on first use; synchronises the plan's stream).
+ * Regions are connected, hold <= 256 vertices each, and are numbered by their smallest seed; the
+ * boundary of a region is its set of vertices with a neighbour in another region. */
+typedef struct {
+  int32_t n_regions;
+  int32_t n_boundary;           /* |B|: the boundary graph's FW runs on this many vertices */
+  int32_t max_region;
+  int32_t max_boundary;         /* largest |B_i| (inner dimension of the products) */
+  int32_t passes;               /* BFS passes (1 + region splits) */
+  int32_t multi_component;      /* G^r has more than one connected component */
+  double sum_region_boundary;   /* sum_i |R_i| |B_i|: the products do N_r times this many min-plus */
+} ear_part_info_t;
+ear_status_t ear_part_info(ear_plan_t plan, ear_part_info_t *info);
 
 /* ---------------------------------------------------------------- Phase III: UPDATE_DISTANCE
  * Alg. 1 lines 9-11 with the rules of sec. 2.1.3: for rows
@@ -349,6 +372,10 @@ typedef struct {
                                   each is also counted in fw16_fallbacks */
   double expand_d16_ms;        /* pair-major expansion: D narrowed to the u16 rows it stages (with the range
                                   check), before the k_expand_pairs launch timed in expand_ms */
+  double part_ms;              /* EAR_FLAG_PART: regions (first solve of a plan), region FWs, boundary FW */
+  double part_mp_ms;           /* EAR_FLAG_PART: the two min-plus products (k_region_mp) */
+  int64_t part_mp_launches;
+  double part_minplus;         /* their algorithmic min-plus: (N_r + |B|) * sum_i |R_i| |B_i| */
 } ear_profile_t;
 
 void ear_profile_enable(int32_t on);

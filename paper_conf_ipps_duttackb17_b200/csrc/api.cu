@@ -175,6 +175,11 @@ ear_status_t apsp_reduced(ear_plan_t p, int32_t *d_D, int64_t ldd, ear_comm_t co
   }
   cudaStream_t st = (cudaStream_t)stream;
   if (!comm) {
+    if (p->flags & EAR_FLAG_PART) {
+      bool applied = false;
+      EAR_TRY(part_rows(p, nullptr, 0, d_D, ldd, Np, &applied, st));
+      if (applied) return EAR_OK;
+    }
     if (p->flags & EAR_FLAG_BCC) return bcc_solve(p, nullptr, d_D, ldd, Np, 0, Np, nullptr, st);
     if (p->flags & EAR_FLAG_SSSP) return sssp_rows(p, d_D, ldd, Np, 0, Np, nullptr, st);
     EAR_TRY(fw_init_D(p, d_D, ldd, Np, 0, Np, st));
@@ -305,7 +310,19 @@ static ear_status_t solve_rows(ear_plan_s *p, int32_t row_begin, int32_t row_end
   const int32_t Np = padded(p, P);
   DKeep k;
   ear_status_t s = EAR_OK;
-  if (!comm && (p->flags & EAR_FLAG_BCC) && u16_ok && xp_applicable(p, st)) {
+  if ((p->flags & EAR_FLAG_PART) && u16_ok && xp_applicable(p, st)) {
+    // Phase II by regions straight into u16 rows; every rank computes all of D (a few ms) and expands
+    // only its own output rows, so no exchange is needed
+    k.ld16 = xp_row_stride(p);
+    EAR_CUDA_TRY(cudaMallocAsync((void **)&k.D16, sizeof(uint16_t) * (size_t)p->n_reduced * k.ld16, st));
+    bool applied = false;
+    s = part_rows(p, k.D16, k.ld16, nullptr, 0, 0, &applied, st);
+    if (s != EAR_OK || !applied) {
+      cudaFreeAsync(k.D16, st);
+      k.D16 = nullptr;
+    }
+  }
+  if (s == EAR_OK && !k.D16 && !comm && (p->flags & EAR_FLAG_BCC) && u16_ok && xp_applicable(p, st)) {
     k.ld16 = xp_row_stride(p);
     int32_t *flag = nullptr;
     EAR_CUDA_TRY(cudaMallocAsync((void **)&k.D16, sizeof(uint16_t) * (size_t)p->n_reduced * k.ld16, st));
@@ -325,7 +342,8 @@ static ear_status_t solve_rows(ear_plan_s *p, int32_t row_begin, int32_t row_end
       k.D16 = nullptr;
     }
   }
-  if (!comm && (p->flags & EAR_FLAG_SSSP) && !(p->flags & EAR_FLAG_BCC) && u16_ok && xp_applicable(p, st)) {
+  if (s == EAR_OK && !k.D16 && !comm && (p->flags & EAR_FLAG_SSSP) && !(p->flags & EAR_FLAG_BCC) && u16_ok &&
+      xp_applicable(p, st)) {
     // per-source SSSP straight into u16 rows: no int32 D, no narrowing pass
     k.ld16 = xp_row_stride(p);
     EAR_CUDA_TRY(cudaMallocAsync((void **)&k.D16, sizeof(uint16_t) * (size_t)p->n_reduced * k.ld16, st));

@@ -49,6 +49,7 @@ struct PeerPtrs {
 
 struct ear_bcc_s;   // bcc.cu: block structure of G^r and the piece layout (EAR_FLAG_BCC)
 struct ear_xp_s;    // expand.cu: the pair-major expansion's item lists (built on first use)
+struct ear_part_s;  // part.cu: the region partition of G^r (EAR_FLAG_PART, built on first use)
 
 // Library-owned plan (Reduce(G) result), device arrays unless noted.
 struct ear_plan_s {
@@ -88,6 +89,7 @@ struct ear_plan_s {
   ear_bcc_s *bcc = nullptr;     // built on first use (EAR_FLAG_BCC, ear_bcc_info)
   int32_t *cc = nullptr;        // [cc_np] connected-component labels of G^r (16-bit FW range check)
   ear_xp_s *xp = nullptr;       // pair-major expansion items (expand.cu), built on first use
+  ear_part_s *part = nullptr;   // region partition (part.cu), built on first use
   int32_t cc_np = 0;
 };
 
@@ -108,7 +110,8 @@ struct ear_comm_s {
 namespace ear {
 // prof.cu
 enum ProfKind { PK_DECOMPOSE, PK_FW_INIT, PK_FW_P1, PK_FW_P2, PK_FW_P3, PK_COMM, PK_EXPAND, PK_SAME_CHAIN, PK_SSSP, PK_BCC, PK_COMPOSE,
-                PK_FW_P3_16, PK_FW16_CONV, PK_FW_SIDE_P1, PK_FW_SIDE_P2, PK_REREDUCE, PK_BCC_PREP, PK_EXPAND_D16 };
+                PK_FW_P3_16, PK_FW16_CONV, PK_FW_SIDE_P1, PK_FW_SIDE_P2, PK_REREDUCE, PK_BCC_PREP, PK_EXPAND_D16,
+                PK_PART, PK_PART_MP };
 void prof_fw16(bool used);   // one 16-bit FW attempt: used, or fell back to int32
 void count_launch(int n = 1);
 int prof_begin(int kind, cudaStream_t s);                // -1 when profiling is off
@@ -186,6 +189,12 @@ ear_status_t bcc_solve(ear_plan_s *plan, ear_comm_s *comm, int32_t *D, int64_t l
                        int32_t rows, const int32_t *d_tile_rows, cudaStream_t stream, uint16_t *D16 = nullptr,
                        int64_t ld16 = 0, int32_t *flag16 = nullptr);
 void bcc_free(ear_bcc_s *b, cudaStream_t stream);
+// part.cu -- Phase II by regions (EAR_FLAG_PART): every row of D as u16 into D16 (ld16 >= round_up(N_r, 8)),
+// or (D16 == NULL) widened into the int32 Np x Np matrix D; *applied = false when the route does not apply
+ear_status_t part_prepare(ear_plan_s *plan, cudaStream_t stream);
+ear_status_t part_rows(ear_plan_s *plan, uint16_t *D16, int64_t ld16, int32_t *D, int64_t ldd, int32_t Np,
+                       bool *applied, cudaStream_t stream);
+void part_free(ear_part_s *q, cudaStream_t stream);
 // expand.cu
 ear_status_t expand(const ear_plan_s *plan, const int32_t *D, int64_t ldd, int32_t row_begin,
                     int32_t row_end, int32_t *out, int64_t ldo, cudaStream_t stream, int prof_kind = PK_EXPAND);

@@ -309,6 +309,8 @@ void plan_free(ear_plan_s *p) {
   p->bcc = nullptr;
   xp_free(p->xp, p->stream);
   p->xp = nullptr;
+  part_free(p->part, p->stream);
+  p->part = nullptr;
   if (p->cc) cudaFreeAsync(p->cc, p->stream);
   p->cc = nullptr;
 }

@@ -1,0 +1,721 @@
+// Phase II by REGIONS: a vertex partition of G^r composed through the region boundaries
+// (EAR_FLAG_PART).  This is sec. 2.2's composition through articulation points (P:129-131,
+// "d(n1, n2) = d(n1, a1) + d(a1, a2) + d(a2, n2)") with the one-vertex separators replaced by the
+// boundary SETS of small regions -- reading C24 in DESIGN.md.
+//
+// Let the vertices of G^r be partitioned into connected regions R_1..R_K, and B_i be the vertices of
+// R_i with a neighbour outside R_i (the boundary), B their union.  d_i is the distance inside the
+// subgraph induced by R_i, d the distance in G^r.  A shortest u-v path (u in R_i) either stays inside
+// R_i, or leaves it for the first time from some b in B_i, so
+//     d(u, v) = min( [v in R_i] d_i(u, v),  min_{b in B_i} d_i(u, b) + d(b, v) )            (1)
+// (every term is the length of a walk, hence >= d(u, v), and the first-exit term is exact).  The same
+// argument on the last entry into R_j gives, for b in B and v in R_j,
+//     d(b, v) = min_{b' in B_j} d(b, b') + d_j(b', v)                                         (2)
+// and the distances between boundary vertices are those of the boundary graph on B with the cliques
+// d_i(b, b') (b, b' in B_i) and the arcs of G^r that join two regions:
+//     d(b, b') = FW over B                                                                     (3)
+// The kernels, in that order:
+//   * k_seed / k_bfs / k_split: regions = Voronoi cells of a multi-source hop BFS (seeds every PSEED
+//     ids plus one vertex per connected component, ties to the smaller seed id), cells larger than
+//     PCAP split again inside themselves with denser seeds -- label-independent up to the seed choice;
+//   * CUB radix sort of (region, boundary-first) keys -> every region's members contiguous, its
+//     boundary first; region / boundary offsets by scans;
+//   * k_region_fw: d_i for every region, one CTA per region, the PCAP x PCAP matrix in registers (8 x 16
+//     entries per thread as packed u16x2, one VIADDMNMX.U16x2 per two min-plus, capped at 0x7FFF);
+//   * the boundary matrix (cliques + joining arcs) and the blocked FW on it (fw_single, packed or int32);
+//   * k_region_mp<false>: (2) for every region j and every boundary column block -> DBVt[v][b] = d(b, v)
+//   * k_region_mp<true>: (1) for every region i and every 128-column block of D -> the u16 rows of D.
+// The two products are min-plus products with the region's boundary as the inner dimension
+// (K = |B_i|, ~10-40 on the paper's sparse graphs): dense work on the ALU pipe at N_r^2 * mean|B_i|
+// min-plus, against the per-source SSSP's N_r * M_r relaxations in hundreds of dependent rounds.
+//
+// Exactness: all distances are integers; the u16 lanes of VIADDMNMX.U16x2 add without saturation, so
+// the route is taken only when no sum of two operands of the same component can reach 0x10000:
+// Dmax + 2 Lmax < 0xFFFF (Lmax the largest d_i, Dmax the largest finite boundary distance).  Sums that
+// involve INF (0xFFFF, other components) wrap, but they only reach entries of pairs in different
+// components, which the last product overwrites with INF.  Otherwise *applied = false and the caller
+// runs another Phase II route.
+#include <cub/cub.cuh>
+
+#include <algorithm>
+#include <climits>
+#include <cstdlib>
+
+#include "common.cuh"
+
+struct ear_part_s {
+  int32_t K = 0, NB = 0, NBp = 0, passes = 0, max_region = 0, max_bnd = 0, multi = 0;
+  double sum_rb = 0;                 // sum over regions of |R_i| |B_i| (product work / N_r)
+  int32_t *reg = nullptr;            // [nr] region of v
+  int32_t *loc = nullptr;            // [nr] index of v inside its region (boundary first)
+  int32_t *perm = nullptr;           // [nr] members of region i at perm[roff[i] .. roff[i+1])
+  int32_t *roff = nullptr;           // [K+1]
+  int32_t *bcnt = nullptr;           // [K] |B_i|
+  int32_t *boff = nullptr;           // [K] first global boundary index of region i
+  int32_t *rcomp = nullptr;          // [K] connected component (cc label) of region i
+  int32_t *bvert = nullptr;          // [NB] vertex of global boundary index g
+  int32_t *gidx = nullptr;           // [nr] global boundary index, -1 inside
+};
+
+namespace ear {
+ear_status_t sssp_prepare(ear_plan_s *p, cudaStream_t st);
+
+namespace {
+
+constexpr int PCAP = 256;            // largest region: its d_i is one CTA's register file
+constexpr int PSEED = 160;           // seed spacing (in vertex ids) of the first Voronoi pass
+constexpr uint32_t PC16 = 0x7FFF;    // cap of the region FW (two capped values never wrap)
+constexpr int FW_NT = 512;
+constexpr int MP_NT = 256, MP_TC = 128, MP_KC = 32, MP_BS = MP_TC + 8;   // Bs row stride (u16): 4-way max
+constexpr int NT = 256;
+
+int grid_n(int64_t n) { return (int)std::max<int64_t>(1, std::min<int64_t>(ceil_div(n, NT), 148 * 16)); }
+
+__device__ __forceinline__ uint32_t dup16(uint32_t x) { return x | (x << 16); }
+
+__global__ void k_seed(const int32_t *__restrict__ cc, int32_t n, int32_t S, int32_t *lab, int32_t *grp) {
+  for (int32_t v = blockIdx.x * blockDim.x + threadIdx.x; v < n; v += gridDim.x * blockDim.x) {
+    lab[v] = (v % S == 0 || cc[v] == v) ? v : -1;
+    grp[v] = 0;
+  }
+}
+
+// one level of the multi-source BFS (Jacobi: an unlabelled vertex takes the smallest label among its
+// neighbours labelled in earlier levels, i.e. of its nearest seeds); only inside its group
+__global__ void k_bfs(const int32_t *__restrict__ rowptr, const int32_t *__restrict__ col, int32_t n,
+                      const int32_t *__restrict__ lin, int32_t *__restrict__ lout, const int32_t *__restrict__ grp,
+                      int32_t *changed) {
+  int ch = 0;
+  for (int32_t v = blockIdx.x * blockDim.x + threadIdx.x; v < n; v += gridDim.x * blockDim.x) {
+    int32_t l = lin[v];
+    if (l < 0) {
+      const int32_t g = grp[v];
+      int32_t m = INT_MAX;
+      for (int32_t a = rowptr[v], e = rowptr[v + 1]; a < e; ++a) {
+        const int32_t u = col[a];
+        const int32_t lu = lin[u];
+        if (lu >= 0 && grp[u] == g) m = min(m, lu);
+      }
+      if (m != INT_MAX) {
+        l = m;
+        ch = 1;
+      }
+    }
+    lout[v] = l;
+  }
+  if (__syncthreads_or(ch) && threadIdx.x == 0) *changed = 1;
+}
+
+__global__ void k_count(const int32_t *__restrict__ lab, int32_t n, int32_t *cnt, int32_t *bad) {
+  for (int32_t v = blockIdx.x * blockDim.x + threadIdx.x; v < n; v += gridDim.x * blockDim.x) {
+    const int32_t l = lab[v];
+    if (l < 0) {
+      *bad = 1;
+      continue;
+    }
+    atomicAdd(&cnt[l], 1);
+  }
+}
+
+// regions above PCAP: their members are unlabelled again except the denser seeds (the old seed and the
+// ids divisible by S2), and grouped by the old region so that the next BFS stays inside it
+__global__ void k_split(int32_t n, int32_t *lab, const int32_t *__restrict__ cnt, int32_t S2, int32_t *grp,
+                        int32_t *over) {
+  int o = 0;
+  for (int32_t v = blockIdx.x * blockDim.x + threadIdx.x; v < n; v += gridDim.x * blockDim.x) {
+    const int32_t l = lab[v];
+    grp[v] = l;
+    if (cnt[l] > PCAP) {
+      lab[v] = (v == l || v % S2 == 0) ? v : -1;
+      o = 1;
+    }
+  }
+  if (__syncthreads_or(o) && threadIdx.x == 0) *over = 1;
+}
+
+__global__ void k_keys(const int32_t *__restrict__ rowptr, const int32_t *__restrict__ col, int32_t n,
+                       const int32_t *__restrict__ lab, uint32_t *keys, int32_t *vals) {
+  for (int32_t v = blockIdx.x * blockDim.x + threadIdx.x; v < n; v += gridDim.x * blockDim.x) {
+    const int32_t l = lab[v];
+    bool bnd = false;
+    for (int32_t a = rowptr[v], e = rowptr[v + 1]; a < e && !bnd; ++a) bnd = lab[col[a]] != l;
+    keys[v] = ((uint32_t)l << 1) | (bnd ? 0u : 1u);
+    vals[v] = v;
+  }
+}
+
+__global__ void k_flags(const uint32_t *__restrict__ sk, int32_t n, int32_t *fstart, int32_t *fbnd) {
+  for (int32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
+    fstart[i] = (i == 0 || (sk[i] >> 1) != (sk[i - 1] >> 1)) ? 1 : 0;
+    fbnd[i] = (sk[i] & 1u) ? 0 : 1;
+  }
+}
+
+// rid = inclusive scan of fstart (region + 1), gpos = exclusive scan of fbnd
+__global__ void k_fill(const int32_t *__restrict__ perm, const int32_t *__restrict__ fstart,
+                       const int32_t *__restrict__ fbnd, const int32_t *__restrict__ rid,
+                       const int32_t *__restrict__ gpos, const int32_t *__restrict__ cc, int32_t n, int32_t *reg,
+                       int32_t *gidx, int32_t *roff, int32_t *boff, int32_t *bcnt, int32_t *rcomp, int32_t *bvert,
+                       int32_t *tot) {
+  for (int32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
+    const int32_t v = perm[i], r = rid[i] - 1;
+    reg[v] = r;
+    if (fstart[i]) {
+      roff[r] = i;
+      boff[r] = gpos[i];
+      rcomp[r] = cc[v];
+    }
+    if (fbnd[i]) {
+      gidx[v] = gpos[i];
+      bvert[gpos[i]] = v;
+      atomicAdd(&bcnt[r], 1);
+    } else {
+      gidx[v] = -1;
+    }
+    if (i == n - 1) {
+      roff[r + 1] = n;
+      tot[0] = r + 1;
+      tot[1] = gpos[i] + fbnd[i];
+    }
+  }
+}
+
+__global__ void k_loc(const int32_t *__restrict__ perm, const int32_t *__restrict__ rid,
+                      const int32_t *__restrict__ roff, int32_t n, int32_t *loc, int32_t *stats) {
+  int mx = 0;
+  for (int32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
+    const int32_t r = rid[i] - 1;
+    loc[perm[i]] = i - roff[r];
+    if (i + 1 == n || rid[i + 1] != rid[i]) mx = max(mx, i + 1 - roff[r]);
+  }
+  for (int o = 16; o; o >>= 1) mx = max(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+  if ((threadIdx.x & 31) == 0 && mx) atomicMax(stats, mx);
+}
+
+// d_i of region i (blockIdx.x): thread (rg, cg) holds rows rg*8..+8, columns cg*16..+16 as 8 x 8 packed
+// pairs; round kk reads row kk (= column kk: d_i is symmetric) from a shared row buffer that the owners
+// of row kk+1 refill after their update -- one barrier per round.  Capped at PC16 (exact below it).
+__global__ void __launch_bounds__(FW_NT, 1)
+    k_region_fw(const int32_t *__restrict__ rowptr, const int32_t *__restrict__ col, const int32_t *__restrict__ w,
+                const int32_t *__restrict__ roff, const int32_t *__restrict__ perm, const int32_t *__restrict__ reg,
+                const int32_t *__restrict__ loc, uint16_t *__restrict__ LR, int32_t *stats) {
+  extern __shared__ __align__(16) uint16_t M[];   // PCAP x PCAP, then two row buffers
+  uint16_t *rowbuf = M + PCAP * PCAP;
+  __shared__ int s_max, s_over;
+  const int i = blockIdx.x, tid = threadIdx.x;
+  const int32_t r0 = roff[i], r = roff[i + 1] - r0, rp = (r + 7) & ~7;
+  if (tid == 0) s_max = 0, s_over = 0;
+  for (int e = tid; e < PCAP * PCAP / 2; e += FW_NT) {
+    const int row = (2 * e) / PCAP, c = (2 * e) % PCAP;
+    reinterpret_cast<uint32_t *>(M)[e] = (row == c ? 0u : PC16) | ((row == c + 1 ? 0u : PC16) << 16);
+  }
+  __syncthreads();
+  int over = 0;
+  for (int a = tid; a < r; a += FW_NT) {
+    const int32_t v = perm[r0 + a];
+    for (int32_t t = rowptr[v], e = rowptr[v + 1]; t < e; ++t) {
+      const int32_t x = col[t];
+      if (reg[x] != i) continue;
+      const int32_t wt = w[t];
+      if (wt >= (int32_t)PC16) over = 1;
+      const int j = loc[x];
+      const uint16_t ww = (uint16_t)min(wt, (int32_t)PC16);
+      if (ww < M[a * PCAP + j]) M[a * PCAP + j] = ww;
+    }
+  }
+  __syncthreads();
+  const int rg = tid >> 4, cg = tid & 15;
+  uint32_t c[8][8];
+#pragma unroll
+  for (int q = 0; q < 8; ++q) {
+    const uint4 *src = reinterpret_cast<const uint4 *>(M + (rg * 8 + q) * PCAP + cg * 16);
+    const uint4 x0 = src[0], x1 = src[1];
+    c[q][0] = x0.x, c[q][1] = x0.y, c[q][2] = x0.z, c[q][3] = x0.w;
+    c[q][4] = x1.x, c[q][5] = x1.y, c[q][6] = x1.z, c[q][7] = x1.w;
+  }
+  if (tid < PCAP / 8) reinterpret_cast<uint4 *>(rowbuf)[tid] = reinterpret_cast<const uint4 *>(M)[tid];
+  __syncthreads();
+  for (int kb = 0; kb < rp / 8; ++kb) {
+#pragma unroll
+    for (int q = 0; q < 8; ++q) {
+      const int kk = kb * 8 + q;
+      const uint16_t *rb = rowbuf + (kk & 1) * PCAP;
+      const uint4 av = *reinterpret_cast<const uint4 *>(rb + rg * 8);
+      const uint4 b0 = *reinterpret_cast<const uint4 *>(rb + cg * 16);
+      const uint4 b1 = *reinterpret_cast<const uint4 *>(rb + cg * 16 + 8);
+      const uint32_t aw[4] = {av.x, av.y, av.z, av.w};
+      const uint32_t b[8] = {b0.x, b0.y, b0.z, b0.w, b1.x, b1.y, b1.z, b1.w};
+#pragma unroll
+      for (int rr = 0; rr < 8; ++rr) {
+        const uint32_t a = dup16((aw[rr >> 1] >> ((rr & 1) * 16)) & 0xFFFFu);
+#pragma unroll
+        for (int p = 0; p < 8; ++p) c[rr][p] = __viaddmin_u16x2(a, b[p], c[rr][p]);
+      }
+      const int nq = (q + 1) & 7;   // compile-time after unrolling
+      if (kk + 1 < rp && rg == kb + (q == 7 ? 1 : 0)) {
+        uint4 *dst = reinterpret_cast<uint4 *>(rowbuf + ((kk + 1) & 1) * PCAP + cg * 16);
+        dst[0] = make_uint4(c[nq][0], c[nq][1], c[nq][2], c[nq][3]);
+        dst[1] = make_uint4(c[nq][4], c[nq][5], c[nq][6], c[nq][7]);
+      }
+      __syncthreads();
+    }
+  }
+  int mx = 0;
+  uint16_t *out = LR + (size_t)i * PCAP * PCAP;
+#pragma unroll
+  for (int q = 0; q < 8; ++q) {
+    const int row = rg * 8 + q;
+    if (row >= rp) continue;
+    uint4 *dst = reinterpret_cast<uint4 *>(out + (size_t)row * PCAP + cg * 16);
+    dst[0] = make_uint4(c[q][0], c[q][1], c[q][2], c[q][3]);
+    dst[1] = make_uint4(c[q][4], c[q][5], c[q][6], c[q][7]);
+    if (row < r) {
+#pragma unroll
+      for (int p = 0; p < 8; ++p)
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+          const int cc = cg * 16 + 2 * p + h;
+          const int x = (c[q][p] >> (16 * h)) & 0xFFFF;
+          if (cc < r) {
+            mx = max(mx, x);
+            if (x >= (int)PC16) over = 1;
+          }
+        }
+    }
+  }
+  __syncthreads();
+  if (mx) atomicMax(&s_max, mx);
+  if (over) s_over = 1;
+  __syncthreads();
+  if (tid == 0) {
+    atomicMax(stats + 0, s_max);
+    if (s_over) atomicOr(stats + 1, 1);
+  }
+}
+
+__global__ void k_bnd_fill(int32_t *dB, int32_t Np) {
+  const int64_t tot = (int64_t)Np * Np;
+  for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < tot; e += (int64_t)gridDim.x * blockDim.x)
+    dB[e] = (e / Np == e % Np) ? 0 : INF;
+}
+
+// the cliques d_i(b, b') of (3), one CTA per region
+__global__ void k_bnd_clique(const uint16_t *__restrict__ LR, const int32_t *__restrict__ bcnt,
+                             const int32_t *__restrict__ boff, int32_t *dB, int32_t ldB) {
+  const int i = blockIdx.x;
+  const int nb = bcnt[i], b0 = boff[i];
+  const uint16_t *L = LR + (size_t)i * PCAP * PCAP;
+  for (int e = threadIdx.x; e < nb * nb; e += blockDim.x) {
+    const int a = e / nb, b = e % nb;
+    const uint32_t x = L[a * PCAP + b];
+    dB[(int64_t)(b0 + a) * ldB + b0 + b] = x >= PC16 ? INF : (int32_t)x;
+  }
+}
+
+// the arcs of G^r that join two regions (both ends are boundary vertices)
+__global__ void k_bnd_cross(const int32_t *__restrict__ rowptr, const int32_t *__restrict__ col,
+                            const int32_t *__restrict__ w, const int32_t *__restrict__ bvert, int32_t NB,
+                            const int32_t *__restrict__ reg, const int32_t *__restrict__ gidx, int32_t *dB,
+                            int32_t ldB) {
+  for (int32_t g = blockIdx.x * blockDim.x + threadIdx.x; g < NB; g += gridDim.x * blockDim.x) {
+    const int32_t v = bvert[g], rv = reg[v];
+    for (int32_t a = rowptr[v], e = rowptr[v + 1]; a < e; ++a) {
+      const int32_t x = col[a];
+      if (reg[x] != rv) atomicMin(&dB[(int64_t)g * ldB + gidx[x]], w[a]);
+    }
+  }
+}
+
+__global__ void k_bnd_lab(const int32_t *__restrict__ bvert, const int32_t *__restrict__ cc, int32_t NB, int32_t Np,
+                          int32_t *labB) {
+  for (int32_t g = blockIdx.x * blockDim.x + threadIdx.x; g < Np; g += gridDim.x * blockDim.x)
+    labB[g] = g < NB ? cc[bvert[g]] : -1 - g;
+}
+
+// u16 copy of the boundary distances (0xFFFF = INF or >= 0xFFFF), and the largest finite one
+__global__ void k_bnd_narrow(const int32_t *__restrict__ dB, int32_t ldB, int32_t NB, int32_t NBp, uint16_t *dB16,
+                             int32_t *stats) {
+  const int64_t tot = (int64_t)NB * (NBp / 2);
+  int mx = 0;
+  for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < tot; e += (int64_t)gridDim.x * blockDim.x) {
+    const int32_t g = (int32_t)(e / (NBp / 2)), h = (int32_t)(e % (NBp / 2)) * 2;
+    uint32_t pr = 0;
+#pragma unroll
+    for (int t = 0; t < 2; ++t) {
+      uint32_t x = 0xFFFFu;
+      if (h + t < NB) {
+        const int32_t d = dB[(int64_t)g * ldB + h + t];
+        if (d < INF) mx = max(mx, d);
+        x = d < 0xFFFF ? (uint32_t)d : 0xFFFFu;
+      }
+      pr |= x << (16 * t);
+    }
+    reinterpret_cast<uint32_t *>(dB16 + (int64_t)g * NBp)[h / 2] = pr;
+  }
+  for (int o = 16; o; o >>= 1) mx = max(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+  if ((threadIdx.x & 31) == 0 && mx) atomicMax(stats, mx);
+}
+
+// Min-plus product of region i (blockIdx.y) with its boundary as the inner dimension, one 128-column
+// block (blockIdx.x) per CTA; thread (rg, cg) owns rows rg*8..+8 and columns cg*16..+16 (8 x 8 pairs).
+//   FINAL = false, (2):  DBVt[v][g] = min_{b < |B_i|} d_i(v, b) + dB16[boff_i + b][g]     (v in R_i)
+//   FINAL = true,  (1):  D16[u][v]  = min( [v in R_i] d_i(u, v), min_b d_i(u, b) + DBVt[v][boff_i + b] ),
+//                        INF when u and v lie in different components (then sums may have wrapped)
+// A = d_i(., B_i) staged per 32-deep chunk as duplicated u32 (row b of the symmetric d_i, coalesced);
+// chunk tails padded with the neutral pair (A = 0xFFFF, B = 0: the sum is 0xFFFF and never wins).
+template <bool FINAL>
+__global__ void __launch_bounds__(MP_NT)
+    k_region_mp(const uint16_t *__restrict__ LR, const int32_t *__restrict__ roff, const int32_t *__restrict__ bcnt,
+                const int32_t *__restrict__ boff, const int32_t *__restrict__ perm, const uint16_t *__restrict__ Bsrc,
+                int64_t ldb, int32_t ncols, uint16_t *__restrict__ out, int64_t ldo, const int32_t *__restrict__ reg,
+                const int32_t *__restrict__ loc, const int32_t *__restrict__ cc, const int32_t *__restrict__ rcomp,
+                int32_t multi) {
+  __shared__ __align__(16) uint32_t As[MP_KC][PCAP];
+  __shared__ __align__(16) uint16_t Bs[MP_KC][MP_BS];
+  __shared__ int32_t cl[MP_TC], ccol[MP_TC];
+  const int i = blockIdx.y, tid = threadIdx.x;
+  const int32_t r0 = roff[i], r = roff[i + 1] - r0, nb = bcnt[i], b0 = boff[i];
+  const int32_t c0 = blockIdx.x * MP_TC;
+  const uint16_t *L = LR + (size_t)i * PCAP * PCAP;
+  const int rg = tid >> 3, cg = tid & 7;
+  if (FINAL && tid < MP_TC) {
+    const int32_t v = c0 + tid;
+    int32_t lc = -1, cv = 0;
+    if (v < ncols) {
+      if (reg[v] == i) lc = loc[v];
+      if (multi) cv = cc[v];
+    }
+    cl[tid] = lc;
+    ccol[tid] = cv;
+  }
+  uint32_t acc[8][8];
+#pragma unroll
+  for (int q = 0; q < 8; ++q)
+#pragma unroll
+    for (int p = 0; p < 8; ++p) acc[q][p] = 0xFFFFFFFFu;
+  const bool active = rg * 8 < r;
+  for (int kb = 0; kb < nb; kb += MP_KC) {
+    const int kc = min(MP_KC, nb - kb), kc8 = (kc + 7) & ~7;
+    __syncthreads();
+    for (int e = tid; e < kc8 * PCAP; e += MP_NT) {
+      const int k = e / PCAP, u = e % PCAP;
+      As[k][u] = (k < kc && u < r) ? dup16(L[(kb + k) * PCAP + u]) : 0xFFFFFFFFu;
+    }
+    if (!FINAL) {
+      for (int e = tid; e < kc8 * (MP_TC / 8); e += MP_NT) {
+        const int k = e / (MP_TC / 8), c8 = (e % (MP_TC / 8)) * 8;
+        uint4 x = make_uint4(0, 0, 0, 0);
+        if (k < kc) x = *reinterpret_cast<const uint4 *>(Bsrc + (int64_t)(b0 + kb + k) * ldb + c0 + c8);
+        *reinterpret_cast<uint4 *>(&Bs[k][c8]) = x;
+      }
+    } else {
+      for (int e = tid; e < kc8 * MP_TC; e += MP_NT) {
+        const int c = e / kc8, k = e % kc8;
+        uint16_t x = 0;
+        if (k < kc) x = c0 + c < ncols ? Bsrc[(int64_t)(c0 + c) * ldb + b0 + kb + k] : (uint16_t)0xFFFF;
+        Bs[k][c] = x;
+      }
+    }
+    __syncthreads();
+    if (active) {
+      for (int k = 0; k < kc8; ++k) {
+        const uint4 a0 = *reinterpret_cast<const uint4 *>(&As[k][rg * 8]);
+        const uint4 a1 = *reinterpret_cast<const uint4 *>(&As[k][rg * 8 + 4]);
+        const uint4 x0 = *reinterpret_cast<const uint4 *>(&Bs[k][cg * 16]);
+        const uint4 x1 = *reinterpret_cast<const uint4 *>(&Bs[k][cg * 16 + 8]);
+        const uint32_t a[8] = {a0.x, a0.y, a0.z, a0.w, a1.x, a1.y, a1.z, a1.w};
+        const uint32_t b[8] = {x0.x, x0.y, x0.z, x0.w, x1.x, x1.y, x1.z, x1.w};
+#pragma unroll
+        for (int q = 0; q < 8; ++q)
+#pragma unroll
+          for (int p = 0; p < 8; ++p) acc[q][p] = __viaddmin_u16x2(a[q], b[p], acc[q][p]);
+      }
+    }
+  }
+  if (FINAL) __syncthreads();   // cl / ccol visible (nb == 0: no barrier in the loop)
+  if (!active) return;
+  const int32_t rc = multi ? rcomp[i] : 0;
+#pragma unroll
+  for (int q = 0; q < 8; ++q) {
+    const int u = rg * 8 + q;
+    if (u >= r) break;
+    const int32_t vu = perm[r0 + u];
+    uint32_t o[8];
+#pragma unroll
+    for (int p = 0; p < 8; ++p) o[p] = acc[q][p];
+    if (FINAL) {
+#pragma unroll
+      for (int p = 0; p < 8; ++p) {
+        uint32_t lo = o[p] & 0xFFFFu, hi = o[p] >> 16;
+        const int ca = cg * 16 + 2 * p;
+        if (cl[ca] >= 0) lo = min(lo, (uint32_t)L[u * PCAP + cl[ca]]);
+        if (cl[ca + 1] >= 0) hi = min(hi, (uint32_t)L[u * PCAP + cl[ca + 1]]);
+        if (c0 + ca >= ncols || (multi && ccol[ca] != rc)) lo = 0xFFFFu;
+        if (c0 + ca + 1 >= ncols || (multi && ccol[ca + 1] != rc)) hi = 0xFFFFu;
+        o[p] = lo | (hi << 16);
+      }
+    }
+    uint16_t *dst = out + (int64_t)vu * ldo + c0 + cg * 16;
+    if (c0 + cg * 16 < ldo) *reinterpret_cast<uint4 *>(dst) = make_uint4(o[0], o[1], o[2], o[3]);
+    if (c0 + cg * 16 + 8 < ldo) *reinterpret_cast<uint4 *>(dst + 8) = make_uint4(o[4], o[5], o[6], o[7]);
+  }
+}
+
+// int32 D (Np x Np, INF, padding isolated) from the u16 rows
+__global__ void k_widen(const uint16_t *__restrict__ D16, int64_t ld16, int32_t nr, int32_t *D, int64_t ldd,
+                        int32_t Np) {
+  const int64_t tot = (int64_t)Np * Np;
+  for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < tot; e += (int64_t)gridDim.x * blockDim.x) {
+    const int32_t r = (int32_t)(e / Np), c = (int32_t)(e % Np);
+    int32_t x;
+    if (r < nr && c < nr) {
+      const uint16_t y = D16[(int64_t)r * ld16 + c];
+      x = y == 0xFFFF ? INF : (int32_t)y;
+    } else {
+      x = r == c ? 0 : INF;
+    }
+    D[(int64_t)r * ldd + c] = x;
+  }
+}
+
+struct Tmp {
+  cudaStream_t st;
+  std::vector<void *> ptrs;
+  explicit Tmp(cudaStream_t s) : st(s) {}
+  ~Tmp() {
+    for (void *p : ptrs) cudaFreeAsync(p, st);
+  }
+  template <typename T>
+  bool get(T **p, size_t n) {
+    if (cudaMallocAsync((void **)p, sizeof(T) * std::max<size_t>(n, 1), st) != cudaSuccess) return false;
+    ptrs.push_back(*p);
+    return true;
+  }
+};
+
+ear_status_t rb1(void *h, const void *d, size_t bytes, cudaStream_t st, const char *what) {
+  Readback rb(st);
+  cudaError_t e = rb.get(h, d, bytes);
+  if (e == cudaSuccess) e = rb.sync();
+  if (e != cudaSuccess) {
+    set_error("%s: %s", what, cudaGetErrorString(e));
+    return EAR_ECUDA;
+  }
+  return EAR_OK;
+}
+
+}  // namespace
+
+void part_free(ear_part_s *q, cudaStream_t st) {
+  if (!q) return;
+  void *a[] = {q->reg, q->loc, q->perm, q->roff, q->bcnt, q->boff, q->rcomp, q->bvert, q->gidx};
+  for (void *x : a)
+    if (x) cudaFreeAsync(x, st);
+  delete q;
+}
+
+// The partition of G^r into regions (cached in the plan).
+ear_status_t part_prepare(ear_plan_s *p, cudaStream_t st) {
+  if (p->part) return EAR_OK;
+  const int32_t n = p->n_reduced;
+  if (n <= 0) {
+    set_error("part_prepare: empty reduced graph");
+    return EAR_EINVAL;
+  }
+  EAR_TRY(sssp_prepare(p, st));
+  const int32_t *cc = nullptr;
+  EAR_TRY(reduced_labels(p, (int32_t)round_up(n, TILE), st, &cc));
+  const int32_t *rowptr = p->r_rowptr, *col = p->r_col;
+  Tmp t(st);
+  int32_t *lab[2], *grp, *cnt, *flags, *rid, *gpos, *fstart, *fbnd, *vals;
+  uint32_t *keys, *skeys;
+  constexpr int NFLAGS = 64;
+  if (!t.get(&lab[0], n) || !t.get(&lab[1], n) || !t.get(&grp, n) || !t.get(&cnt, n) || !t.get(&flags, NFLAGS) ||
+      !t.get(&rid, n) || !t.get(&gpos, n) || !t.get(&fstart, n) || !t.get(&fbnd, n) || !t.get(&vals, n) ||
+      !t.get(&keys, n) || !t.get(&skeys, n)) {
+    set_error("part_prepare: out of device memory");
+    return EAR_ENOMEM;
+  }
+  ear_part_s *q = new ear_part_s();
+  auto fail = [&](ear_status_t s) {
+    part_free(q, st);
+    return s;
+  };
+  const int g = grid_n(n);
+  EAR_LAUNCH(k_seed, g, NT, 0, st)(cc, n, PSEED, lab[0], grp);
+  int cur = 0, passes = 0;
+  for (int32_t S2 = PSEED / 2;; S2 = std::max(1, S2 / 2)) {
+    // BFS levels in batches of 8 launches, one readback per batch
+    for (int it = 0;; it += 8) {
+      EAR_CUDA_TRY(dev_memset(flags, 0, 8 * sizeof(int32_t), st));
+      for (int b = 0; b < 8; ++b) {
+        EAR_LAUNCH(k_bfs, g, NT, 0, st)(rowptr, col, n, lab[cur], lab[cur ^ 1], grp, flags + b);
+        cur ^= 1;
+      }
+      int32_t h[8];
+      ear_status_t s = rb1(h, flags, sizeof(h), st, "part_prepare");
+      if (s != EAR_OK) return fail(s);
+      if (!h[7]) break;
+      if (it > 4 * n) return fail((set_error("part_prepare: BFS did not converge"), EAR_ECUDA));
+    }
+    ++passes;
+    EAR_CUDA_TRY(dev_memset(cnt, 0, sizeof(int32_t) * n, st));
+    EAR_CUDA_TRY(dev_memset(flags, 0, 2 * sizeof(int32_t), st));
+    EAR_LAUNCH(k_count, g, NT, 0, st)(lab[cur], n, cnt, flags);
+    EAR_LAUNCH(k_split, g, NT, 0, st)(n, lab[cur], cnt, S2, grp, flags + 1);
+    int32_t h[2];
+    ear_status_t s = rb1(h, flags, sizeof(h), st, "part_prepare");
+    if (s != EAR_OK) return fail(s);
+    if (h[0]) return fail((set_error("part_prepare: unlabelled vertex after the BFS"), EAR_ECUDA));
+    if (!h[1]) break;
+    if (passes > 12) return fail((set_error("part_prepare: region splitting did not converge"), EAR_ECUDA));
+  }
+  q->passes = passes;
+  // members by (region, boundary first, id)
+  EAR_LAUNCH(k_keys, g, NT, 0, st)(rowptr, col, n, lab[cur], keys, vals);
+  if (cudaMallocAsync((void **)&q->perm, sizeof(int32_t) * n, st) != cudaSuccess)
+    return fail((set_error("part_prepare: out of device memory"), EAR_ENOMEM));
+  int bits = 1;
+  while ((int64_t)1 << bits < 2 * (int64_t)n) ++bits;
+  size_t tb1 = 0, tb2 = 0, tb3 = 0;
+  cub::DeviceRadixSort::SortPairs(nullptr, tb1, keys, skeys, vals, q->perm, n, 0, bits, st);
+  cub::DeviceScan::InclusiveSum(nullptr, tb2, fstart, rid, n, st);
+  cub::DeviceScan::ExclusiveSum(nullptr, tb3, fbnd, gpos, n, st);
+  void *tmp = nullptr;
+  if (!t.get((char **)&tmp, std::max({tb1, tb2, tb3})))
+    return fail((set_error("part_prepare: out of device memory"), EAR_ENOMEM));
+  EAR_CUDA_TRY(cub::DeviceRadixSort::SortPairs(tmp, tb1, keys, skeys, vals, q->perm, n, 0, bits, st));
+  EAR_LAUNCH(k_flags, g, NT, 0, st)(skeys, n, fstart, fbnd);
+  EAR_CUDA_TRY(cub::DeviceScan::InclusiveSum(tmp, tb2, fstart, rid, n, st));
+  EAR_CUDA_TRY(cub::DeviceScan::ExclusiveSum(tmp, tb3, fbnd, gpos, n, st));
+  // region count K <= n; allocate the per-region arrays for n (small) and fill
+  auto need = [&](int32_t **x, size_t m) { return cudaMallocAsync((void **)x, sizeof(int32_t) * std::max<size_t>(m, 1), st); };
+  if (need(&q->reg, n) || need(&q->loc, n) || need(&q->gidx, n) || need(&q->roff, (size_t)n + 1) ||
+      need(&q->boff, n) || need(&q->bcnt, n) || need(&q->rcomp, n) || need(&q->bvert, n))
+    return fail((set_error("part_prepare: out of device memory"), EAR_ENOMEM));
+  EAR_CUDA_TRY(dev_memset(q->bcnt, 0, sizeof(int32_t) * n, st));
+  EAR_CUDA_TRY(dev_memset(flags, 0, 4 * sizeof(int32_t), st));
+  EAR_LAUNCH(k_fill, g, NT, 0, st)(q->perm, fstart, fbnd, rid, gpos, cc, n, q->reg, q->gidx, q->roff, q->boff, q->bcnt,
+                                   q->rcomp, q->bvert, flags);
+  EAR_LAUNCH(k_loc, g, NT, 0, st)(q->perm, rid, q->roff, n, q->loc, flags + 2);
+  int32_t h[4];
+  {
+    ear_status_t s = rb1(h, flags, sizeof(h), st, "part_prepare");
+    if (s != EAR_OK) return fail(s);
+  }
+  q->K = h[0];
+  q->NB = h[1];
+  q->max_region = h[2];
+  q->NBp = (int32_t)round_up(std::max(q->NB, 1), MP_TC);
+  // host copies of the small per-region counts (statistics: max |B_i|, sum |R_i||B_i|, components)
+  std::vector<int32_t> hro(q->K + 1), hbc(q->K), hrc(q->K);
+  EAR_CUDA_TRY(cudaMemcpyAsync(hro.data(), q->roff, sizeof(int32_t) * (q->K + 1), cudaMemcpyDeviceToHost, st));
+  EAR_CUDA_TRY(cudaMemcpyAsync(hbc.data(), q->bcnt, sizeof(int32_t) * q->K, cudaMemcpyDeviceToHost, st));
+  EAR_CUDA_TRY(cudaMemcpyAsync(hrc.data(), q->rcomp, sizeof(int32_t) * q->K, cudaMemcpyDeviceToHost, st));
+  EAR_CUDA_TRY(cudaStreamSynchronize(st));
+  q->sum_rb = 0;
+  q->max_bnd = 0;
+  for (int i = 0; i < q->K; ++i) {
+    q->sum_rb += (double)(hro[i + 1] - hro[i]) * hbc[i];
+    q->max_bnd = std::max(q->max_bnd, hbc[i]);
+    if (hrc[i] != hrc[0]) q->multi = 1;
+  }
+  p->part = q;
+  EAR_CUDA_TRY(cudaGetLastError());
+  return EAR_OK;
+}
+
+// Every row of D (reduced vertex order) as u16 (0xFFFF = INF, stride ld16 >= round_up(N_r, 8)), or
+// -- with D (int32, Np x Np, ldd) -- widened into it.  *applied = false when the route does not apply
+// (too many regions, a region distance or a sum that could reach 0xFFFF); nothing is written then.
+ear_status_t part_rows(ear_plan_s *p, uint16_t *D16, int64_t ld16, int32_t *D, int64_t ldd, int32_t Np, bool *applied,
+                       cudaStream_t st) {
+  *applied = false;
+  const int32_t n = p->n_reduced;
+  if (n <= 0) return EAR_OK;
+  int ps = prof_begin(PK_PART, st);
+  EAR_TRY(part_prepare(p, st));
+  ear_part_s *q = p->part;
+  // mostly tiny components (K near N_r): the (column blocks x regions) product grid would dominate
+  if (q->K > n / 16 && (double)q->K * ceil_div(n, MP_TC) > 65536.0) {
+    prof_end(ps, st, 0);
+    return EAR_OK;
+  }
+  Tmp t(st);
+  uint16_t *LR = nullptr, *dB16 = nullptr, *DBVt = nullptr, *own16 = nullptr;
+  int32_t *dB = nullptr, *labB = nullptr, *stats = nullptr;
+  const int32_t NB = q->NB, NBp = q->NBp, NpB = (int32_t)round_up(std::max(NB, 1), TILE);
+  if (!t.get(&LR, (size_t)q->K * PCAP * PCAP) || !t.get(&stats, 4) || !t.get(&dB, (size_t)NpB * NpB) ||
+      !t.get(&labB, NpB) || !t.get(&dB16, (size_t)std::max(NB, 1) * NBp) || !t.get(&DBVt, (size_t)n * NBp)) {
+    set_error("part_rows: out of device memory");
+    return EAR_ENOMEM;
+  }
+  EAR_CUDA_TRY(dev_memset(stats, 0, 4 * sizeof(int32_t), st));
+  const int fw_smem = (PCAP * PCAP + 2 * PCAP) * (int)sizeof(uint16_t);
+  EAR_CUDA_TRY(smem_attr((const void *)k_region_fw, fw_smem));
+  EAR_LAUNCH(k_region_fw, q->K, FW_NT, fw_smem, st)(p->r_rowptr, p->r_col, p->r_w, q->roff, q->perm, q->reg, q->loc, LR,
+                                                     stats);
+  // (3): the boundary graph and its FW
+  EAR_LAUNCH(k_bnd_fill, grid_n((int64_t)NpB * NpB), NT, 0, st)(dB, NpB);
+  EAR_LAUNCH(k_bnd_clique, q->K, NT, 0, st)(LR, q->bcnt, q->boff, dB, NpB);
+  if (NB > 0) {
+    EAR_LAUNCH(k_bnd_cross, grid_n(NB), NT, 0, st)(p->r_rowptr, p->r_col, p->r_w, q->bvert, NB, q->reg, q->gidx, dB,
+                                                   NpB);
+    const int32_t *cc = nullptr;
+    EAR_TRY(reduced_labels(p, (int32_t)round_up(n, TILE), st, &cc));
+    EAR_LAUNCH(k_bnd_lab, grid_n(NpB), NT, 0, st)(q->bvert, cc, NB, NpB, labB);
+    EAR_TRY(fw_single(dB, NpB, NpB, st, labB, NB, !(p->flags & EAR_FLAG_FW32), nullptr));
+    EAR_LAUNCH(k_bnd_narrow, grid_n((int64_t)NB * NBp / 2), NT, 0, st)(dB, NpB, NB, NBp, dB16, stats + 2);
+  }
+  int32_t h[4];
+  EAR_TRY(rb1(h, stats, sizeof(h), st, "part_rows"));
+  const int64_t Lmax = h[0], Dmax = h[2];
+  prof_end(ps, st, 0);
+  if (h[1] || Dmax + 2 * Lmax >= 0xFFFF) return EAR_OK;
+  const int32_t *cc = nullptr;
+  if (q->multi) EAR_TRY(reduced_labels(p, (int32_t)round_up(n, TILE), st, &cc));
+  int pm = prof_begin(PK_PART_MP, st);
+  if (NB > 0) {
+    dim3 g1(NBp / MP_TC, q->K);
+    EAR_LAUNCH(k_region_mp<false>, g1, MP_NT, 0, st)(LR, q->roff, q->bcnt, q->boff, q->perm, dB16, NBp, NBp, DBVt, NBp,
+                                                      q->reg, q->loc, cc, q->rcomp, q->multi);
+  }
+  uint16_t *out = D16;
+  int64_t ldo = ld16;
+  if (!out) {
+    ldo = round_up(n, 8);
+    if (!t.get(&own16, (size_t)n * ldo)) {
+      set_error("part_rows: out of device memory");
+      return EAR_ENOMEM;
+    }
+    out = own16;
+  }
+  dim3 g2((unsigned)ceil_div(ldo, MP_TC), q->K);
+  EAR_LAUNCH(k_region_mp<true>, g2, MP_NT, 0, st)(LR, q->roff, q->bcnt, q->boff, q->perm, DBVt, NBp, n, out, ldo,
+                                                   q->reg, q->loc, cc, q->rcomp, q->multi);
+  prof_end(pm, st, (double)n * q->sum_rb + (double)NB * q->sum_rb);
+  if (D) EAR_LAUNCH(k_widen, grid_n((int64_t)Np * Np), NT, 0, st)(out, ldo, n, D, ldd, Np);
+  EAR_CUDA_TRY(cudaGetLastError());
+  *applied = true;
+  return EAR_OK;
+}
+
+}  // namespace ear
+
+extern "C" ear_status_t ear_part_info(ear_plan_t p, ear_part_info_t *info) {
+  using namespace ear;
+  if (!p || !info) {
+    set_error("ear_part_info: NULL argument");
+    return EAR_EINVAL;
+  }
+  EAR_TRY(part_prepare(p, p->stream));
+  const ear_part_s *q = p->part;
+  info->n_regions = q->K;
+  info->n_boundary = q->NB;
+  info->max_region = q->max_region;
+  info->max_boundary = q->max_bnd;
+  info->passes = q->passes;
+  info->multi_component = q->multi;
+  info->sum_region_boundary = q->sum_rb;
+  return EAR_OK;
+}

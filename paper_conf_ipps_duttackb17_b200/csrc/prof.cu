@@ -260,6 +260,8 @@ ear_status_t ear_profile_read(ear_profile_t *out) {
       case PK_REREDUCE: g_acc.rereduce_ms += ms; break;
       case PK_BCC_PREP: g_acc.bcc_prepare_ms += ms; break;
       case PK_EXPAND_D16: g_acc.expand_d16_ms += ms; break;
+      case PK_PART: g_acc.part_ms += ms; break;
+      case PK_PART_MP: g_acc.part_mp_ms += ms; g_acc.part_mp_launches++; g_acc.part_minplus += r.work; break;
       default: break;
     }
     g_pool.push_back(r.e0);

@@ -29,6 +29,7 @@ FLAG_NO_CONTRACT = 1
 FLAG_SSSP = 2
 FLAG_BCC = 4
 FLAG_FW32 = 8
+FLAG_PART = 16
 
 _lib = None
 
@@ -57,7 +58,9 @@ class _Profile(ctypes.Structure):
                 ("fw16_conv_ms", ctypes.c_double), ("fw_phase3_16_ms", ctypes.c_double),
                 ("fw_phase3_16_minplus", ctypes.c_double), ("fw_side_ms", ctypes.c_double),
                 ("rereduce_ms", ctypes.c_double), ("bcc_prepare_ms", ctypes.c_double),
-                ("fw16_prechecked", ctypes.c_int64), ("expand_d16_ms", ctypes.c_double)]
+                ("fw16_prechecked", ctypes.c_int64), ("expand_d16_ms", ctypes.c_double),
+                ("part_ms", ctypes.c_double), ("part_mp_ms", ctypes.c_double), ("part_mp_launches", ctypes.c_int64),
+                ("part_minplus", ctypes.c_double)]
 
 
 class _BccInfo(ctypes.Structure):
@@ -65,6 +68,12 @@ class _BccInfo(ctypes.Structure):
                 ("n_pieces", ctypes.c_int32), ("largest_piece", ctypes.c_int32), ("tree_levels", ctypes.c_int32),
                 ("sum_cubes", ctypes.c_double), ("rereduced_pieces", ctypes.c_int32), ("largest_reduced", ctypes.c_int32),
                 ("rereduce_levels", ctypes.c_int32)]
+
+
+class _PartInfo(ctypes.Structure):
+    _fields_ = [("n_regions", ctypes.c_int32), ("n_boundary", ctypes.c_int32), ("max_region", ctypes.c_int32),
+                ("max_boundary", ctypes.c_int32), ("passes", ctypes.c_int32), ("multi_component", ctypes.c_int32),
+                ("sum_region_boundary", ctypes.c_double)]
 
 
 class _McbInfo(ctypes.Structure):
@@ -82,6 +91,7 @@ SIGNATURES = {
     "ear_plan_export_reduced_edges": (_I32, [_P, _P, _P, _P, _P]),
     "ear_plan_destroy": (None, [_P]),
     "ear_bcc_info": (_I32, [_P, ctypes.POINTER(_BccInfo)]),
+    "ear_part_info": (_I32, [_P, ctypes.POINTER(_PartInfo)]),
     "apsp_reduced": (_I32, [_P, _P, _I64, _P, _P]),
     "apsp_reduced_emulated": (_I32, [_P, _I32, _P, _I64, _P]),
     "apsp_reduced_rank_timing": (_I32, [_P, _I32, _I32, _P]),
@@ -241,6 +251,12 @@ class Plan:
         i = _BccInfo()
         _check(lib().ear_bcc_info(self.handle, ctypes.byref(i)), "ear_bcc_info")
         return {f: getattr(i, f) for f, _ in _BccInfo._fields_}
+
+    def part_info(self) -> dict:
+        """Region partition of G^r used by FLAG_PART (ear_part_info; builds it on first use, synchronises)."""
+        i = _PartInfo()
+        _check(lib().ear_part_info(self.handle, ctypes.byref(i)), "ear_part_info")
+        return {f: getattr(i, f) for f, _ in _PartInfo._fields_}
 
     def export(self, stream=None) -> dict:
         """Per-vertex descriptors as CUDA int32 tensors (tests)."""
