@@ -5,18 +5,22 @@
 
 One step = one pass of the whole hot path over the workload: apsp_full =
 Reduce(G) chain contraction -> Phase II on G^r -> ear expansion of this rank's rows of the N x N int32
-matrix, graph already resident in HBM.  By default (--phase2 bcc_sssp) Phase II splits G^r into its
-biconnected pieces (paper sec. 2.2), reduces every big piece again and solves it by
-the paper's own per-source SSSP (near-far rounds on u16 shared-memory rows), joining the pieces
-through the articulation points; --phase2 bcc solves the pieces by the blocked min-plus FW, --phase2 fw
-runs one FW over all of G^r, --phase2 sssp the SSSP over all of G^r.  For N > 1 GPUs (torchrun, one
-process per GPU) the largest piece's rows are split over the ranks and every rank expands its own row
-block; the total work is fixed (strong scaling).  Timing: W untimed warm-up steps, then exactly K
-steps between barrier + synchronize, CUDA events on the launching stream, max over ranks.  The output
-(40 GB) is far larger than L2, so no flush is needed between steps.
+matrix, graph already resident in HBM.  By default (--phase2 part) Phase II cuts G^r into connected
+regions of <= 256 vertices and composes every row of D through the region boundaries (sec. 2.2's
+composition through articulation points, with boundary sets as separators):
+region distances by one CTA each, a blocked FW on the boundary graph, two min-plus products with a
+region boundary as the inner dimension.  --phase2 bcc_sssp splits G^r into its biconnected pieces
+(P:119-131), reduces every big piece again and solves it by the paper's own per-source SSSP
+(P:101); --phase2 bcc solves the pieces by the blocked min-plus FW, --phase2 fw runs one FW over all of
+G^r, --phase2 sssp the SSSP over all of G^r.  For N > 1 GPUs (torchrun, one process per GPU) every rank
+computes D (a few ms) and expands its own row block; the total work is fixed (strong scaling).  Timing:
+W untimed warm-up steps, then exactly K steps between barrier + synchronize, CUDA events on the
+launching stream, max over ranks.  The output (40 GB) is far larger than L2, so no flush is needed
+between steps.
 
-Rank 0 prints one JSON line.  Extra keys: roofline (dominant kernel: the per-source SSSP, or the FW
-phase-3 min-plus tile kernel on the FW routes), roofline_expand (HBM bound), cpu_baseline (the CPU oracle on a bounded sample,
+Rank 0 prints one JSON line.  Extra keys: roofline (the kernel with the largest share of the step: the
+expansion k_expand_pairs, HBM bound, on the region route; else the Phase II kernel), roofline_phase2 /
+roofline_expand (the other one), cpu_baseline (the CPU oracle on a bounded sample,
 rank 0 at N = 1 only), e2e (the same metric through the host-buffer C-ABI calls with every step's
 H2D edge upload and D2H copy of the output rows: by default K jobs of apsp_full_host_async pipelined one
 deep -- job i+1's Phases I-II overlap job i's expansion and row copies -- into two pinned output buffers;
@@ -417,6 +421,16 @@ def run_ours(args, rank, world, local_rank):
               "bcc_prepare": prof["bcc_prepare_ms"] / K, "expand_d16": prof["expand_d16_ms"] / K,
               "fw_side_overlapped": prof["fw_side_ms"] / K}
     fw_minplus = prof["fw_phase2_minplus"] + prof["fw_phase3_minplus"]
+    # "roofline" = the kernel with the largest share of the step (the expansion once Phase II runs by
+    # regions); the other one is reported beside it
+    phase2_ms = (prof["part_mp_ms"] if args.phase2 == "part" else prof["sssp_ms"] if args.phase2 in ("sssp", "bcc_sssp")
+                 else p3_ms)
+    roofline["step_share"] = phase2_ms / K / (profiled_ms or 1.0)
+    roofline_expand["step_share"] = ex_ms / K / (profiled_ms or 1.0)
+    if ex_ms >= phase2_ms:
+        rooflines = {"roofline": roofline_expand, "roofline_phase2": roofline}
+    else:
+        rooflines = {"roofline": roofline, "roofline_expand": roofline_expand}
     del out
     torch.cuda.empty_cache()
 
@@ -527,6 +541,8 @@ def run_ours(args, rank, world, local_rank):
                 "ms_per_step": ms_max / K, "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
                 "dtype": ("int32 (SSSP: u16 shared-memory rows, exact below 0xFFFF; int32 fallback)"
                           if args.phase2 in ("sssp", "bcc_sssp") else
+                          "int32 (regions: packed u16x2 min-plus, exact while Dmax + 2 Lmax < 0xFFFF; other routes "
+                          "otherwise)" if args.phase2 == "part" else
                           "int32" if prof["fw16_used"] == 0 else "int32 (FW: packed u16x2, exact below 0x7FFF)"),
                 "data": "synthetic (seeded generator, spatially coherent labels)",
                 "fw16": {"used": int(prof["fw16_used"]) // K, "fallbacks": int(prof["fw16_fallbacks"]) // K},
@@ -538,7 +554,7 @@ def run_ours(args, rank, world, local_rank):
                            "phase2": args.phase2, "bcc": bcc, "part": part,
                            "l2": "inputs larger than L2 (D %.1f GB, output %.1f GB per step)" % (
                                4.0 * info.n_reduced_padded ** 2 / 1e9, 4.0 * g.n * g.n / 1e9)},
-                "roofline": roofline, "roofline_expand": roofline_expand,
+                **rooflines,
                 "fw_minplus_gops": fw_minplus / (fw_ms / 1e3) / 1e9 if fw_ms > 0 else None,
                 "phases_ms": phases, "phase2_alternatives": alt, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks,
                 "gpu_launches": launches, "step_ms": step_ms, "seeds": seeds,
@@ -560,7 +576,7 @@ def main():
     ap.add_argument("--config", default="cfg4")
     ap.add_argument("--seed", type=int, default=0)
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
-    ap.add_argument("--phase2", choices=["part", "bcc_sssp", "bcc", "fw", "sssp"], default="bcc_sssp",
+    ap.add_argument("--phase2", choices=["part", "bcc_sssp", "bcc", "fw", "sssp"], default="part",
                     help="Phase II: the biconnected pieces of G^r (paper sec. 2.2) each reduced again and solved by "
                          "per-source SSSP (the paper's own Phase II, P:101; default), the same pieces by blocked FW, "
                          "blocked FW on all of G^r, or per-source SSSP on all of G^r")

@@ -55,10 +55,22 @@ struct ear_part_s {
   int32_t *rcomp = nullptr;          // [K] connected component (cc label) of region i
   int32_t *bvert = nullptr;          // [NB] vertex of global boundary index g
   int32_t *gidx = nullptr;           // [nr] global boundary index, -1 inside
+  int32_t *big = nullptr;            // [nbig] regions with |B_i| > MP_KC (the general product kernel)
+  int32_t nbig = 0;
+  int32_t *itemoff = nullptr;        // [K+1] first k_region_final item of region i (tiles of W_i columns)
+  int64_t items_ld = -1;             // the row length the item offsets were cut for
+  std::vector<int32_t> h_roff, h_bcnt;
 };
 
 namespace ear {
 ear_status_t sssp_prepare(ear_plan_s *p, cudaStream_t st);
+
+// a graph as the region route reads it: CSR (both arc directions, parallel arcs merged), and connected-
+// component labels that are the smallest vertex id of the component
+struct GView {
+  int32_t n;
+  const int32_t *rowptr, *col, *w, *cc;
+};
 
 namespace {
 
@@ -68,6 +80,8 @@ constexpr uint32_t PC16 = 0x7FFF;    // cap of the region FW (two capped values 
 constexpr int FW_NT = 512;
 constexpr int MP_NT = 256, MP_TC = 128, MP_KC = 32, MP_BS = MP_TC + 8;   // Bs row stride (u16): 4-way max
 constexpr int NT = 256;
+constexpr int PREC_MIN = 1024;      // a boundary graph this large is solved by regions again
+constexpr int PREC_DEPTH = 2;       // ... down to this nesting depth (then by the blocked FW)
 
 int grid_n(int64_t n) { return (int)std::max<int64_t>(1, std::min<int64_t>(ceil_div(n, NT), 148 * 16)); }
 
@@ -369,11 +383,11 @@ __global__ void __launch_bounds__(MP_NT)
                 const int32_t *__restrict__ boff, const int32_t *__restrict__ perm, const uint16_t *__restrict__ Bsrc,
                 int64_t ldb, int32_t ncols, uint16_t *__restrict__ out, int64_t ldo, const int32_t *__restrict__ reg,
                 const int32_t *__restrict__ loc, const int32_t *__restrict__ cc, const int32_t *__restrict__ rcomp,
-                int32_t multi) {
+                int32_t multi, const int32_t *__restrict__ rlist) {
   __shared__ __align__(16) uint32_t As[MP_KC][PCAP];
   __shared__ __align__(16) uint16_t Bs[MP_KC][MP_BS];
   __shared__ int32_t cl[MP_TC], ccol[MP_TC];
-  const int i = blockIdx.y, tid = threadIdx.x;
+  const int i = rlist ? rlist[blockIdx.y] : blockIdx.y, tid = threadIdx.x;
   const int32_t r0 = roff[i], r = roff[i + 1] - r0, nb = bcnt[i], b0 = boff[i];
   const int32_t c0 = blockIdx.x * MP_TC;
   const uint16_t *L = LR + (size_t)i * PCAP * PCAP;
@@ -461,6 +475,237 @@ __global__ void __launch_bounds__(MP_NT)
   }
 }
 
+// DBV[g][v] = DBVt[v][g]: the boundary rows of d as the final product stages them (rows contiguous in v)
+constexpr int TR = 64;
+__global__ void k_transpose16(const uint16_t *__restrict__ in, int64_t ldi, int32_t rows, int32_t cols,
+                              uint16_t *__restrict__ out, int64_t ldo) {
+  __shared__ uint16_t tile[TR][TR + 2];
+  const int r0 = blockIdx.y * TR, c0 = blockIdx.x * TR;
+  for (int e = threadIdx.x; e < TR * TR; e += blockDim.x) {
+    const int r = e / TR, c = e % TR;
+    if (r0 + r < rows && c0 + c < cols) tile[r][c] = in[(int64_t)(r0 + r) * ldi + c0 + c];
+  }
+  __syncthreads();
+  for (int e = threadIdx.x; e < TR * TR; e += blockDim.x) {
+    const int c = e / TR, r = e % TR;
+    if (r0 + r < rows && c0 + c < cols) out[(int64_t)(c0 + c) * ldo + r0 + r] = tile[r][c];
+  }
+}
+
+__device__ __forceinline__ void cp_async16(void *smem, const void *gmem, int bytes) {
+  const uint32_t s = (uint32_t)__cvta_generic_to_shared(smem);
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;\n" ::"r"(s), "l"(gmem), "r"(bytes));
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::); }
+__device__ __forceinline__ void cp_async_wait1() { asm volatile("cp.async.wait_group 1;\n" ::: "memory"); }
+
+// (1) for the regions with |B_i| <= MP_KC, persistent.  The tile of region i is its r_i rows x W_i
+// columns, W_i = 16 * min(32, 256 / ceil(r_i / 8)) (every thread busy whatever the region size: thread
+// (ro, cg) owns rows ro*8..+8 and columns cg*16..+16); a CTA walks a contiguous range of (region, tile)
+// items in region-major order, so A = d_i(., B_i) is staged once per region, and the B rows (DBV rows of
+// B_i, contiguous in v) of the next tile stream into the other half of a double buffer by cp.async while
+// the current tile is computed.  Tiles without a vertex of the region skip the local-term checks.
+constexpr int FW_MAXW = 512, FW_BS = FW_MAXW + 8;
+__global__ void __launch_bounds__(MP_NT, 2)
+    k_region_final(const uint16_t *__restrict__ LR, const int32_t *__restrict__ roff, const int32_t *__restrict__ bcnt,
+                   const int32_t *__restrict__ boff, const int32_t *__restrict__ perm,
+                   const uint16_t *__restrict__ DBV, int64_t ldv, int32_t n, uint16_t *__restrict__ out, int64_t ldo,
+                   const int32_t *__restrict__ reg, const int32_t *__restrict__ loc, const int32_t *__restrict__ cc,
+                   const int32_t *__restrict__ rcomp, int32_t multi, const int32_t *__restrict__ itemoff, int32_t K) {
+  extern __shared__ __align__(16) uint8_t smraw[];
+  uint32_t(*As)[PCAP] = reinterpret_cast<uint32_t(*)[PCAP]>(smraw);                                // [MP_KC][PCAP]
+  uint16_t(*Bs)[MP_KC][FW_BS] = reinterpret_cast<uint16_t(*)[MP_KC][FW_BS]>(smraw + MP_KC * PCAP * 4);  // [2]
+  __shared__ int32_t cl[FW_MAXW], ccol[FW_MAXW];
+  const int tid = threadIdx.x;
+  const int32_t total = itemoff[K];
+  const int32_t t0 = (int32_t)((int64_t)total * blockIdx.x / gridDim.x);
+  const int32_t t1 = (int32_t)((int64_t)total * (blockIdx.x + 1) / gridDim.x);
+  if (t0 >= t1) return;
+  // region of item t: itemoff is monotone, items are visited in order
+  int ri = 0;
+  {
+    int lo = 0, hi = K - 1;
+    while (lo < hi) {
+      const int mid = (lo + hi + 1) >> 1;
+      if (itemoff[mid] <= t0) lo = mid; else hi = mid - 1;
+    }
+    ri = lo;
+  }
+  auto width_of = [&](int32_t r) { return 16 * min(32, MP_NT / max(1, (r + 7) >> 3)); };
+  auto issue = [&](int32_t t, int i, int buf) {
+    const int32_t r = roff[i + 1] - roff[i], nb = bcnt[i], b0 = boff[i];
+    const int32_t W = width_of(r), c0 = (t - itemoff[i]) * W;
+    const int chunks = W / 8;
+    for (int e = tid; e < nb * chunks; e += MP_NT) {
+      const int k = e / chunks, c8 = (e % chunks) * 8;
+      const bool ok = c0 + c8 < ldv;
+      cp_async16(&Bs[buf][k][c8], DBV + (int64_t)(b0 + k) * ldv + (ok ? c0 + c8 : 0), ok ? 16 : 0);
+    }
+    cp_async_commit();
+  };
+  int cur = -1, buf = 0;
+  issue(t0, ri, 0);
+  for (int32_t t = t0; t < t1; ++t) {
+    while (itemoff[ri + 1] <= t) ++ri;
+    const int i = ri;
+    const int32_t r0 = roff[i], r = roff[i + 1] - r0, nb = bcnt[i];
+    const int32_t nro = (r + 7) >> 3, W = width_of(r), cgs = W / 16, c0 = (t - itemoff[i]) * W;
+    __syncthreads();   // tile t-1 is done with As, Bs[buf ^ 1], cl
+    if (i != cur) {
+      cur = i;
+      const uint16_t *L = LR + (size_t)i * PCAP * PCAP;
+      for (int e = tid; e < nb * PCAP; e += MP_NT) {
+        const int k = e / PCAP, u = e % PCAP;
+        As[k][u] = u < r ? dup16(L[k * PCAP + u]) : 0xFFFFFFFFu;
+      }
+    }
+    int loc_any = 0;
+    for (int c = tid; c < W; c += MP_NT) {
+      const int32_t v = c0 + c;
+      int32_t lc = -1, cv = 0;
+      if (v < n) {
+        if (reg[v] == i) lc = loc[v];
+        if (multi) cv = cc[v];
+      }
+      cl[c] = lc;
+      ccol[c] = cv;
+      loc_any |= lc >= 0;
+    }
+    if (t + 1 < t1) {
+      int in = ri;
+      while (itemoff[in + 1] <= t + 1) ++in;
+      issue(t + 1, in, buf ^ 1);
+    } else {
+      cp_async_commit();   // keep the group count uniform
+    }
+    cp_async_wait1();
+    loc_any = __syncthreads_or(loc_any);
+    const int cgi = tid % cgs, ro = tid / cgs;
+    if (ro < nro) {
+      uint32_t acc[8][8];
+#pragma unroll
+      for (int q = 0; q < 8; ++q)
+#pragma unroll
+        for (int p = 0; p < 8; ++p) acc[q][p] = 0xFFFFFFFFu;
+      const uint16_t *bsrc = &Bs[buf][0][cgi * 16];
+      for (int k = 0; k < nb; ++k) {
+        const uint4 a0 = *reinterpret_cast<const uint4 *>(&As[k][ro * 8]);
+        const uint4 a1 = *reinterpret_cast<const uint4 *>(&As[k][ro * 8 + 4]);
+        const uint4 x0 = *reinterpret_cast<const uint4 *>(bsrc + k * FW_BS);
+        const uint4 x1 = *reinterpret_cast<const uint4 *>(bsrc + k * FW_BS + 8);
+        const uint32_t a[8] = {a0.x, a0.y, a0.z, a0.w, a1.x, a1.y, a1.z, a1.w};
+        const uint32_t b[8] = {x0.x, x0.y, x0.z, x0.w, x1.x, x1.y, x1.z, x1.w};
+#pragma unroll
+        for (int q = 0; q < 8; ++q)
+#pragma unroll
+          for (int p = 0; p < 8; ++p) acc[q][p] = __viaddmin_u16x2(a[q], b[p], acc[q][p]);
+      }
+      const uint16_t *L = LR + (size_t)i * PCAP * PCAP;
+      const int rc = multi ? rcomp[i] : 0;
+      const bool fix = loc_any || multi || c0 + W > n;
+      const int cb = c0 + cgi * 16;
+#pragma unroll
+      for (int q = 0; q < 8; ++q) {
+        const int u = ro * 8 + q;
+        if (u < r) {
+          uint32_t o[8];
+#pragma unroll
+          for (int p = 0; p < 8; ++p) o[p] = acc[q][p];
+          if (fix) {
+#pragma unroll
+            for (int p = 0; p < 8; ++p) {
+              uint32_t lo = o[p] & 0xFFFFu, hi = o[p] >> 16;
+              const int ca = cgi * 16 + 2 * p;
+              if (cl[ca] >= 0) lo = min(lo, (uint32_t)L[u * PCAP + cl[ca]]);
+              if (cl[ca + 1] >= 0) hi = min(hi, (uint32_t)L[u * PCAP + cl[ca + 1]]);
+              if (c0 + ca >= n || (multi && ccol[ca] != rc)) lo = 0xFFFFu;
+              if (c0 + ca + 1 >= n || (multi && ccol[ca + 1] != rc)) hi = 0xFFFFu;
+              o[p] = lo | (hi << 16);
+            }
+          }
+          uint16_t *dst = out + (int64_t)perm[r0 + u] * ldo + cb;
+          if (cb < ldo) *reinterpret_cast<uint4 *>(dst) = make_uint4(o[0], o[1], o[2], o[3]);
+          if (cb + 8 < ldo) *reinterpret_cast<uint4 *>(dst + 8) = make_uint4(o[4], o[5], o[6], o[7]);
+        }
+      }
+    }
+    buf ^= 1;
+  }
+}
+constexpr int FINAL_SMEM = MP_KC * PCAP * 4 + 2 * MP_KC * FW_BS * 2;
+
+// The boundary graph H of a level: vertex g = global boundary index; arcs: the clique of its region's
+// boundary with weights d_i (local indices: the boundary comes first in a region) and its joining arcs.
+__global__ void k_h_deg(const int32_t *__restrict__ rowptr, const int32_t *__restrict__ col,
+                        const int32_t *__restrict__ bvert, int32_t NB, const int32_t *__restrict__ reg,
+                        const int32_t *__restrict__ bcnt, int32_t *deg) {
+  for (int32_t g = blockIdx.x * blockDim.x + threadIdx.x; g <= NB; g += gridDim.x * blockDim.x) {
+    if (g == NB) {
+      deg[g] = 0;
+      continue;
+    }
+    const int32_t v = bvert[g], i = reg[v];
+    int32_t d = bcnt[i] - 1;
+    for (int32_t a = rowptr[v], e = rowptr[v + 1]; a < e; ++a) d += reg[col[a]] != i;
+    deg[g] = d;
+  }
+}
+
+__global__ void k_h_fill(const int32_t *__restrict__ rowptr, const int32_t *__restrict__ col,
+                         const int32_t *__restrict__ w, const int32_t *__restrict__ bvert, int32_t NB,
+                         const int32_t *__restrict__ reg, const int32_t *__restrict__ gidx,
+                         const int32_t *__restrict__ bcnt, const int32_t *__restrict__ boff,
+                         const uint16_t *__restrict__ LR, const int32_t *__restrict__ hrow, int32_t *hcol, int32_t *hw) {
+  for (int32_t g = blockIdx.x * blockDim.x + threadIdx.x; g < NB; g += gridDim.x * blockDim.x) {
+    const int32_t v = bvert[g], i = reg[v], b0 = boff[i], nb = bcnt[i], a = g - b0;
+    const uint16_t *L = LR + (size_t)i * PCAP * PCAP + (size_t)a * PCAP;
+    int32_t pos = hrow[g];
+    for (int32_t b = 0; b < nb; ++b) {
+      if (b == a) continue;
+      hcol[pos] = b0 + b;
+      hw[pos] = L[b];
+      ++pos;
+    }
+    for (int32_t t = rowptr[v], e = rowptr[v + 1]; t < e; ++t) {
+      const int32_t x = col[t];
+      if (reg[x] == i) continue;
+      hcol[pos] = gidx[x];
+      hw[pos] = w[t];
+      ++pos;
+    }
+  }
+}
+
+// components of H are those of the graph restricted to its boundary (a component with two or more regions
+// has all its boundary vertices connected through the cliques and joining arcs); label = smallest g.
+// Two passes: hcc == nullptr -> mn[cc] = min g; else hcc[g] = mn[cc(g)]
+__global__ void k_h_cc(const int32_t *__restrict__ bvert, const int32_t *__restrict__ cc, int32_t NB, int32_t *mn,
+                       int32_t *hcc) {
+  for (int32_t g = blockIdx.x * blockDim.x + threadIdx.x; g < NB; g += gridDim.x * blockDim.x) {
+    const int32_t c = cc[bvert[g]];
+    if (hcc) hcc[g] = mn[c];
+    else atomicMin(&mn[c], g);
+  }
+}
+
+// largest entry < 0xFFFF of a u16 matrix (rows x ld, ld % 8 == 0)
+__global__ void k_max16(const uint16_t *__restrict__ M, int32_t rows, int64_t ld, int32_t *out) {
+  const int64_t tot = (int64_t)rows * (ld / 8);
+  uint32_t mx = 0;
+  for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < tot; e += (int64_t)gridDim.x * blockDim.x) {
+    const uint4 v = reinterpret_cast<const uint4 *>(M)[e];
+    const uint32_t w4[4] = {v.x, v.y, v.z, v.w};
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const uint32_t lo = w4[j] & 0xFFFFu, hi = w4[j] >> 16;
+      if (lo != 0xFFFFu) mx = max(mx, lo);
+      if (hi != 0xFFFFu) mx = max(mx, hi);
+    }
+  }
+  for (int o = 16; o; o >>= 1) mx = max(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+  if ((threadIdx.x & 31) == 0 && mx) atomicMax(out, (int32_t)mx);
+}
+
 // int32 D (Np x Np, INF, padding isolated) from the u16 rows
 __global__ void k_widen(const uint16_t *__restrict__ D16, int64_t ld16, int32_t nr, int32_t *D, int64_t ldd,
                         int32_t Np) {
@@ -508,24 +753,17 @@ ear_status_t rb1(void *h, const void *d, size_t bytes, cudaStream_t st, const ch
 
 void part_free(ear_part_s *q, cudaStream_t st) {
   if (!q) return;
-  void *a[] = {q->reg, q->loc, q->perm, q->roff, q->bcnt, q->boff, q->rcomp, q->bvert, q->gidx};
+  void *a[] = {q->reg, q->loc, q->perm, q->roff, q->bcnt, q->boff, q->rcomp, q->bvert, q->gidx, q->big, q->itemoff};
   for (void *x : a)
     if (x) cudaFreeAsync(x, st);
   delete q;
 }
 
-// The partition of G^r into regions (cached in the plan).
-ear_status_t part_prepare(ear_plan_s *p, cudaStream_t st) {
-  if (p->part) return EAR_OK;
-  const int32_t n = p->n_reduced;
-  if (n <= 0) {
-    set_error("part_prepare: empty reduced graph");
-    return EAR_EINVAL;
-  }
-  EAR_TRY(sssp_prepare(p, st));
-  const int32_t *cc = nullptr;
-  EAR_TRY(reduced_labels(p, (int32_t)round_up(n, TILE), st, &cc));
-  const int32_t *rowptr = p->r_rowptr, *col = p->r_col;
+// The partition of a graph into regions (G^r: cached in the plan; the boundary graph: per solve).
+ear_status_t part_build(const GView &gv, cudaStream_t st, ear_part_s **out) {
+  *out = nullptr;
+  const int32_t n = gv.n;
+  const int32_t *rowptr = gv.rowptr, *col = gv.col, *cc = gv.cc;
   Tmp t(st);
   int32_t *lab[2], *grp, *cnt, *flags, *rid, *gpos, *fstart, *fbnd, *vals;
   uint32_t *keys, *skeys;
@@ -615,88 +853,194 @@ ear_status_t part_prepare(ear_plan_s *p, cudaStream_t st) {
   EAR_CUDA_TRY(cudaStreamSynchronize(st));
   q->sum_rb = 0;
   q->max_bnd = 0;
+  q->h_roff = hro;
+  q->h_bcnt = hbc;
+  std::vector<int32_t> big;
   for (int i = 0; i < q->K; ++i) {
     q->sum_rb += (double)(hro[i + 1] - hro[i]) * hbc[i];
     q->max_bnd = std::max(q->max_bnd, hbc[i]);
     if (hrc[i] != hrc[0]) q->multi = 1;
+    if (hbc[i] > MP_KC) big.push_back(i);
   }
-  p->part = q;
+  q->nbig = (int32_t)big.size();
+  if (!big.empty()) {
+    if (cudaMallocAsync((void **)&q->big, sizeof(int32_t) * big.size(), st) != cudaSuccess)
+      return fail((set_error("part_prepare: out of device memory"), EAR_ENOMEM));
+    EAR_CUDA_TRY(cudaMemcpyAsync(q->big, big.data(), sizeof(int32_t) * big.size(), cudaMemcpyHostToDevice, st));
+    EAR_CUDA_TRY(cudaStreamSynchronize(st));
+  }
+  *out = q;
   EAR_CUDA_TRY(cudaGetLastError());
   return EAR_OK;
 }
 
-// Every row of D (reduced vertex order) as u16 (0xFFFF = INF, stride ld16 >= round_up(N_r, 8)), or
-// -- with D (int32, Np x Np, ldd) -- widened into it.  *applied = false when the route does not apply
-// (too many regions, a region distance or a sum that could reach 0xFFFF); nothing is written then.
-ear_status_t part_rows(ear_plan_s *p, uint16_t *D16, int64_t ld16, int32_t *D, int64_t ldd, int32_t Np, bool *applied,
-                       cudaStream_t st) {
-  *applied = false;
-  const int32_t n = p->n_reduced;
-  if (n <= 0) return EAR_OK;
-  int ps = prof_begin(PK_PART, st);
-  EAR_TRY(part_prepare(p, st));
-  ear_part_s *q = p->part;
-  // mostly tiny components (K near N_r): the (column blocks x regions) product grid would dominate
-  if (q->K > n / 16 && (double)q->K * ceil_div(n, MP_TC) > 65536.0) {
-    prof_end(ps, st, 0);
-    return EAR_OK;
+static ear_status_t plan_view(ear_plan_s *p, cudaStream_t st, GView *gv) {
+  EAR_TRY(sssp_prepare(p, st));
+  const int32_t *cc = nullptr;
+  EAR_TRY(reduced_labels(p, (int32_t)round_up(p->n_reduced, TILE), st, &cc));
+  *gv = GView{p->n_reduced, p->r_rowptr, p->r_col, p->r_w, cc};
+  return EAR_OK;
+}
+
+ear_status_t part_prepare(ear_plan_s *p, cudaStream_t st) {
+  if (p->part) return EAR_OK;
+  if (p->n_reduced <= 0) {
+    set_error("part_prepare: empty reduced graph");
+    return EAR_EINVAL;
   }
+  GView gv;
+  EAR_TRY(plan_view(p, st, &gv));
+  return part_build(gv, st, &p->part);
+}
+
+// Every row of the view's distance matrix as u16 (0xFFFF = INF, row stride ldo >= round_up(n, 8)) into
+// out.  depth: nesting level (the boundary graph of a level is solved by the same route when it is big).
+// *applied = false when the route does not apply (too many regions, a region distance or a sum that
+// could reach 0xFFFF); nothing is written then.  Profiled (PK_PART / PK_PART_MP) at depth 0 only.
+ear_status_t part_solve(const GView &gv, ear_part_s *q, uint16_t *out, int64_t ldo, int depth, bool fw32,
+                        bool *applied, cudaStream_t st) {
+  *applied = false;
+  const int32_t n = gv.n;
+  // mostly tiny components (K near n): the (column blocks x regions) product grid would dominate
+  if (q->K > n / 16 && (double)q->K * ceil_div(n, MP_TC) > 65536.0) return EAR_OK;
+  const int ps = depth == 0 ? prof_begin(PK_PART, st) : -1;
   Tmp t(st);
-  uint16_t *LR = nullptr, *dB16 = nullptr, *DBVt = nullptr, *own16 = nullptr;
-  int32_t *dB = nullptr, *labB = nullptr, *stats = nullptr;
-  const int32_t NB = q->NB, NBp = q->NBp, NpB = (int32_t)round_up(std::max(NB, 1), TILE);
-  if (!t.get(&LR, (size_t)q->K * PCAP * PCAP) || !t.get(&stats, 4) || !t.get(&dB, (size_t)NpB * NpB) ||
-      !t.get(&labB, NpB) || !t.get(&dB16, (size_t)std::max(NB, 1) * NBp) || !t.get(&DBVt, (size_t)n * NBp)) {
-    set_error("part_rows: out of device memory");
+  uint16_t *LR = nullptr, *dB16 = nullptr, *DBVt = nullptr, *DBV = nullptr;
+  int32_t *stats = nullptr;
+  const int32_t NB = q->NB, NBp = q->NBp;
+  if (!t.get(&LR, (size_t)q->K * PCAP * PCAP) || !t.get(&stats, 4) || !t.get(&dB16, (size_t)std::max(NB, 1) * NBp) ||
+      !t.get(&DBVt, (size_t)n * NBp)) {
+    set_error("part_solve: out of device memory");
     return EAR_ENOMEM;
   }
   EAR_CUDA_TRY(dev_memset(stats, 0, 4 * sizeof(int32_t), st));
   const int fw_smem = (PCAP * PCAP + 2 * PCAP) * (int)sizeof(uint16_t);
   EAR_CUDA_TRY(smem_attr((const void *)k_region_fw, fw_smem));
-  EAR_LAUNCH(k_region_fw, q->K, FW_NT, fw_smem, st)(p->r_rowptr, p->r_col, p->r_w, q->roff, q->perm, q->reg, q->loc, LR,
+  EAR_LAUNCH(k_region_fw, q->K, FW_NT, fw_smem, st)(gv.rowptr, gv.col, gv.w, q->roff, q->perm, q->reg, q->loc, LR,
                                                      stats);
-  // (3): the boundary graph and its FW
-  EAR_LAUNCH(k_bnd_fill, grid_n((int64_t)NpB * NpB), NT, 0, st)(dB, NpB);
-  EAR_LAUNCH(k_bnd_clique, q->K, NT, 0, st)(LR, q->bcnt, q->boff, dB, NpB);
+  // (3): distances between boundary vertices
   if (NB > 0) {
-    EAR_LAUNCH(k_bnd_cross, grid_n(NB), NT, 0, st)(p->r_rowptr, p->r_col, p->r_w, q->bvert, NB, q->reg, q->gidx, dB,
-                                                   NpB);
-    const int32_t *cc = nullptr;
-    EAR_TRY(reduced_labels(p, (int32_t)round_up(n, TILE), st, &cc));
-    EAR_LAUNCH(k_bnd_lab, grid_n(NpB), NT, 0, st)(q->bvert, cc, NB, NpB, labB);
-    EAR_TRY(fw_single(dB, NpB, NpB, st, labB, NB, !(p->flags & EAR_FLAG_FW32), nullptr));
-    EAR_LAUNCH(k_bnd_narrow, grid_n((int64_t)NB * NBp / 2), NT, 0, st)(dB, NpB, NB, NBp, dB16, stats + 2);
+    bool done = false;
+    if (depth < PREC_DEPTH && NB >= PREC_MIN) {
+      // the boundary graph H (cliques d_i on every B_i + the joining arcs) by the same route
+      Tmp th(st);
+      int32_t *hdeg, *hrow, *hcol, *hw, *hcc, *mn;
+      size_t tb = 0;
+      cub::DeviceScan::ExclusiveSum(nullptr, tb, (int32_t *)nullptr, (int32_t *)nullptr, NB + 1, st);
+      void *tmp = nullptr;
+      if (!th.get(&hdeg, (size_t)NB + 1) || !th.get(&hrow, (size_t)NB + 1) || !th.get(&hcc, NB) ||
+          !th.get(&mn, n) || !th.get((char **)&tmp, tb)) {
+        set_error("part_solve: out of device memory");
+        return EAR_ENOMEM;
+      }
+      EAR_LAUNCH(k_h_deg, grid_n(NB + 1), NT, 0, st)(gv.rowptr, gv.col, q->bvert, NB, q->reg, q->bcnt, hdeg);
+      EAR_CUDA_TRY(cub::DeviceScan::ExclusiveSum(tmp, tb, hdeg, hrow, NB + 1, st));
+      int32_t arcs = 0;
+      EAR_TRY(rb1(&arcs, hrow + NB, sizeof(int32_t), st, "part_solve"));
+      if (!th.get(&hcol, arcs) || !th.get(&hw, arcs)) {
+        set_error("part_solve: out of device memory");
+        return EAR_ENOMEM;
+      }
+      EAR_LAUNCH(k_h_fill, grid_n(NB), NT, 0, st)(gv.rowptr, gv.col, gv.w, q->bvert, NB, q->reg, q->gidx, q->bcnt, q->boff,
+                                                  LR, hrow, hcol, hw);
+      EAR_CUDA_TRY(dev_memset(mn, 0x7F, sizeof(int32_t) * n, st));
+      EAR_LAUNCH(k_h_cc, grid_n(NB), NT, 0, st)(q->bvert, gv.cc, NB, mn, nullptr);
+      EAR_LAUNCH(k_h_cc, grid_n(NB), NT, 0, st)(q->bvert, gv.cc, NB, mn, hcc);
+      const GView hv{NB, hrow, hcol, hw, hcc};
+      ear_part_s *qh = nullptr;
+      EAR_TRY(part_build(hv, st, &qh));
+      ear_status_t s = part_solve(hv, qh, dB16, NBp, depth + 1, fw32, &done, st);
+      part_free(qh, st);
+      EAR_TRY(s);
+      if (done) EAR_LAUNCH(k_max16, grid_n((int64_t)NB * NBp / 8), NT, 0, st)(dB16, NB, NBp, stats + 2);
+    }
+    if (!done) {   // dense: blocked FW over the boundary matrix
+      int32_t *dB = nullptr, *labB = nullptr;
+      const int32_t NpB = (int32_t)round_up(NB, TILE);
+      if (!t.get(&dB, (size_t)NpB * NpB) || !t.get(&labB, NpB)) {
+        set_error("part_solve: out of device memory");
+        return EAR_ENOMEM;
+      }
+      EAR_LAUNCH(k_bnd_fill, grid_n((int64_t)NpB * NpB), NT, 0, st)(dB, NpB);
+      EAR_LAUNCH(k_bnd_clique, q->K, NT, 0, st)(LR, q->bcnt, q->boff, dB, NpB);
+      EAR_LAUNCH(k_bnd_cross, grid_n(NB), NT, 0, st)(gv.rowptr, gv.col, gv.w, q->bvert, NB, q->reg, q->gidx, dB, NpB);
+      EAR_LAUNCH(k_bnd_lab, grid_n(NpB), NT, 0, st)(q->bvert, gv.cc, NB, NpB, labB);
+      EAR_TRY(fw_single(dB, NpB, NpB, st, labB, NB, !fw32, nullptr));
+      EAR_LAUNCH(k_bnd_narrow, grid_n((int64_t)NB * NBp / 2), NT, 0, st)(dB, NpB, NB, NBp, dB16, stats + 2);
+    }
   }
   int32_t h[4];
-  EAR_TRY(rb1(h, stats, sizeof(h), st, "part_rows"));
+  EAR_TRY(rb1(h, stats, sizeof(h), st, "part_solve"));
   const int64_t Lmax = h[0], Dmax = h[2];
-  prof_end(ps, st, 0);
+  if (ps >= 0) prof_end(ps, st, 0);
   if (h[1] || Dmax + 2 * Lmax >= 0xFFFF) return EAR_OK;
-  const int32_t *cc = nullptr;
-  if (q->multi) EAR_TRY(reduced_labels(p, (int32_t)round_up(n, TILE), st, &cc));
-  int pm = prof_begin(PK_PART_MP, st);
+  const int32_t *cc = q->multi ? gv.cc : nullptr;
+  const int pm = depth == 0 ? prof_begin(PK_PART_MP, st) : -1;
+  const int64_t ldv = round_up(n, 8);
   if (NB > 0) {
     dim3 g1(NBp / MP_TC, q->K);
     EAR_LAUNCH(k_region_mp<false>, g1, MP_NT, 0, st)(LR, q->roff, q->bcnt, q->boff, q->perm, dB16, NBp, NBp, DBVt, NBp,
-                                                      q->reg, q->loc, cc, q->rcomp, q->multi);
+                                                      q->reg, q->loc, cc, q->rcomp, q->multi, nullptr);
+    if (!t.get(&DBV, (size_t)NB * ldv)) {
+      set_error("part_solve: out of device memory");
+      return EAR_ENOMEM;
+    }
+    dim3 gt((unsigned)ceil_div(NB, TR), (unsigned)ceil_div(n, TR));
+    EAR_LAUNCH(k_transpose16, gt, NT, 0, st)(DBVt, NBp, n, NB, DBV, ldv);
   }
+  if (q->items_ld != ldo) {   // tiles of W_i columns per region (regions with a big boundary: none)
+    std::vector<int32_t> off(q->K + 1, 0);
+    for (int i = 0; i < q->K; ++i) {
+      const int32_t r = q->h_roff[i + 1] - q->h_roff[i];
+      const int32_t W = 16 * std::min(32, MP_NT / std::max(1, (r + 7) >> 3));
+      off[i + 1] = off[i] + (q->h_bcnt[i] > MP_KC ? 0 : (int32_t)ceil_div(n, W));
+    }
+    if (!q->itemoff && cudaMallocAsync((void **)&q->itemoff, sizeof(int32_t) * (q->K + 1), st) != cudaSuccess) {
+      set_error("part_solve: out of device memory");
+      return EAR_ENOMEM;
+    }
+    EAR_CUDA_TRY(cudaMemcpyAsync(q->itemoff, off.data(), sizeof(int32_t) * (q->K + 1), cudaMemcpyHostToDevice, st));
+    EAR_CUDA_TRY(cudaStreamSynchronize(st));
+    q->items_ld = ldo;
+  }
+  EAR_CUDA_TRY(smem_attr((const void *)k_region_final, FINAL_SMEM));
+  EAR_LAUNCH(k_region_final, 2 * num_sms(), MP_NT, FINAL_SMEM, st)(LR, q->roff, q->bcnt, q->boff, q->perm, DBV, ldv, n,
+                                                                    out, ldo, q->reg, q->loc, cc, q->rcomp, q->multi,
+                                                                    q->itemoff, q->K);
+  if (q->nbig > 0) {
+    dim3 g2((unsigned)ceil_div(ldo, MP_TC), q->nbig);
+    EAR_LAUNCH(k_region_mp<true>, g2, MP_NT, 0, st)(LR, q->roff, q->bcnt, q->boff, q->perm, DBVt, NBp, n, out, ldo,
+                                                     q->reg, q->loc, cc, q->rcomp, q->multi, q->big);
+  }
+  if (pm >= 0) prof_end(pm, st, (double)n * q->sum_rb + (double)NB * q->sum_rb);
+  EAR_CUDA_TRY(cudaGetLastError());
+  *applied = true;
+  return EAR_OK;
+}
+
+// Every row of D (reduced vertex order) as u16 (0xFFFF = INF, stride ld16 >= round_up(N_r, 8)), or
+// -- with D (int32, Np x Np, ldd) -- widened into it.  *applied = false when the route does not apply.
+ear_status_t part_rows(ear_plan_s *p, uint16_t *D16, int64_t ld16, int32_t *D, int64_t ldd, int32_t Np, bool *applied,
+                       cudaStream_t st) {
+  *applied = false;
+  const int32_t n = p->n_reduced;
+  if (n <= 0) return EAR_OK;
+  EAR_TRY(part_prepare(p, st));
+  GView gv;
+  EAR_TRY(plan_view(p, st, &gv));
+  Tmp t(st);
   uint16_t *out = D16;
   int64_t ldo = ld16;
   if (!out) {
     ldo = round_up(n, 8);
-    if (!t.get(&own16, (size_t)n * ldo)) {
+    if (!t.get(&out, (size_t)n * ldo)) {
       set_error("part_rows: out of device memory");
       return EAR_ENOMEM;
     }
-    out = own16;
   }
-  dim3 g2((unsigned)ceil_div(ldo, MP_TC), q->K);
-  EAR_LAUNCH(k_region_mp<true>, g2, MP_NT, 0, st)(LR, q->roff, q->bcnt, q->boff, q->perm, DBVt, NBp, n, out, ldo,
-                                                   q->reg, q->loc, cc, q->rcomp, q->multi);
-  prof_end(pm, st, (double)n * q->sum_rb + (double)NB * q->sum_rb);
-  if (D) EAR_LAUNCH(k_widen, grid_n((int64_t)Np * Np), NT, 0, st)(out, ldo, n, D, ldd, Np);
+  EAR_TRY(part_solve(gv, p->part, out, ldo, 0, (p->flags & EAR_FLAG_FW32) != 0, applied, st));
+  if (*applied && D) EAR_LAUNCH(k_widen, grid_n((int64_t)Np * Np), NT, 0, st)(out, ldo, n, D, ldd, Np);
   EAR_CUDA_TRY(cudaGetLastError());
-  *applied = true;
   return EAR_OK;
 }
 

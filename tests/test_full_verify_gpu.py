@@ -1,7 +1,7 @@
 """Full N x N verification at the north-star sizes (S defined at P:109; SURVEY 8.c pin P4).
 
 Every entry of cfg4's matrix (100k vertices, 40 GB) in the bench's launch configuration (apsp_full,
-Phase II by biconnected pieces solved by per-source SSSP) and by the blocked-FW route, and -- with EAR_VERIFY_CFG5=1 -- every entry of cfg5's (200k vertices,
+Phase II by regions, EAR_FLAG_PART), by biconnected pieces solved by per-source SSSP and by the blocked-FW route, and -- with EAR_VERIFY_CFG5=1 -- every entry of cfg5's (200k vertices,
 160 GB: Phase II once, the expansion in row blocks) is checked by the oracle's Bellman certificate
 (oracle.certify_rows: the definition of S restated as a fixed point whose only solution is S) on the
 host's cores, streaming row blocks device -> pinned host while the previous block is being certified.
@@ -73,7 +73,8 @@ def report(summary):
     print(json.dumps(summary))
 
 
-ROUTES = {"bcc_sssp": ("FLAG_BCC | FLAG_SSSP (bench default)", lambda ea: ea.FLAG_BCC | ea.FLAG_SSSP),
+ROUTES = {"part": ("FLAG_PART (regions; bench default)", lambda ea: ea.FLAG_PART | ea.FLAG_BCC | ea.FLAG_SSSP),
+          "bcc_sssp": ("FLAG_BCC | FLAG_SSSP", lambda ea: ea.FLAG_BCC | ea.FLAG_SSSP),
           "bcc_fw": ("FLAG_BCC (pieces by the blocked FW)", lambda ea: ea.FLAG_BCC)}
 
 

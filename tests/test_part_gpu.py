@@ -173,3 +173,21 @@ def test_row_range(pkg):
     out, ran = run(pkg, g, rows=(1234, 5678))
     assert ran
     exact(out.cpu().numpy(), oracle.apsp_rows(g.n, g.src, g.dst, g.w, np.arange(1234, 5678)), "rows")
+
+
+@pytest.mark.parametrize("n,deg", [(1500, 3), (3000, 4)])
+def test_expander_big_boundaries(pkg, n, deg):
+    """a random sparse graph (an expander: most region vertices are boundary vertices, |B_i| > 32, so the
+    general product kernel runs beside the persistent one)"""
+    rng = np.random.default_rng(n)
+    m = n * deg // 2
+    src = rng.integers(0, n, m).astype(np.int32)
+    dst = rng.integers(0, n, m).astype(np.int32)
+    ring = np.arange(n, dtype=np.int32)   # connected
+    g = Graph(n, np.r_[src, ring], np.r_[dst, (ring + 1) % n].astype(np.int32),
+              rng.integers(1, 101, m + n).astype(np.int32))
+    pi, _ = part_info(pkg, g)
+    assert pi["max_boundary"] > 32
+    out, ran = run(pkg, g)
+    exact(out.cpu().numpy(), oracle.apsp(g.n, g.src, g.dst, g.w), f"expander n={n}")
+    assert ran

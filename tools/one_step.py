@@ -1,4 +1,4 @@
-"""One apsp_full call on a config (for ncu launch lists): python tools/one_step.py cfg4 [bcc_sssp|bcc|sssp|fw]"""
+"""One apsp_full call on a config (for ncu launch lists): python tools/one_step.py cfg4 [part|bcc_sssp|bcc|sssp|fw]"""
 import sys
 import time
 
@@ -10,7 +10,8 @@ from paper_conf_ipps_duttackb17_b200 import graphgen as gg  # noqa: E402
 
 cfg = sys.argv[1] if len(sys.argv) > 1 else "cfg4"
 route = sys.argv[2] if len(sys.argv) > 2 else "bcc_sssp"
-flags = {"bcc_sssp": ea.FLAG_BCC | ea.FLAG_SSSP, "bcc": ea.FLAG_BCC, "sssp": ea.FLAG_SSSP, "fw": 0}[route]
+flags = {"bcc_sssp": ea.FLAG_BCC | ea.FLAG_SSSP, "bcc": ea.FLAG_BCC, "sssp": ea.FLAG_SSSP, "fw": 0,
+         "part": ea.FLAG_PART | ea.FLAG_BCC | ea.FLAG_SSSP}[route]
 g = gg.config(cfg)
 src, dst, w = (torch.as_tensor(x).cuda() for x in (g.src, g.dst, g.w))
 out = torch.empty((g.n, g.n), dtype=torch.int32, device="cuda")
