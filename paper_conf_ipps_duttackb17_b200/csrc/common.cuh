@@ -90,6 +90,7 @@ struct ear_plan_s {
   int32_t *cc = nullptr;        // [cc_np] connected-component labels of G^r (16-bit FW range check)
   ear_xp_s *xp = nullptr;       // pair-major expansion items (expand.cu), built on first use
   ear_part_s *part = nullptr;   // region partition (part.cu), built on first use
+  int32_t connected = -1;       // G^r has one connected component: 1 / 0, -1 unknown (set with the partition)
   int32_t cc_np = 0;
 };
 

@@ -364,20 +364,35 @@ __device__ __forceinline__ int32_t d16(const uint16_t *row, uint32_t t) {
   const uint32_t x = row[t];
   return x == 0xFFFFu ? INF : (int32_t)x;
 }
+// R[j] = min(D[row, p_t] + cp_t, D[row, q_t] + cq_t) for the 4 columns; CONN: G^r is connected, so no
+// entry of D is INF (0xFFFF) and no clamping is needed
+template <bool CONN>
 __device__ __forceinline__ void r_of(const uint16_t *row, const uint32_t pq[4], const uint32_t cc[4], int32_t R[4]) {
 #pragma unroll
-  for (int j = 0; j < 4; ++j)
-    R[j] = min(__viaddmin_s32(d16(row, pq[j] >> 16), (int32_t)(cc[j] >> 16), d16(row, pq[j] & 0xFFFFu) + (int32_t)(cc[j] & 0xFFFFu)), INF);
+  for (int j = 0; j < 4; ++j) {
+    if (CONN)
+      R[j] = __viaddmin_s32((int32_t)row[pq[j] >> 16], (int32_t)(cc[j] >> 16),
+                            (int32_t)row[pq[j] & 0xFFFFu] + (int32_t)(cc[j] & 0xFFFFu));
+    else
+      R[j] = min(__viaddmin_s32(d16(row, pq[j] >> 16), (int32_t)(cc[j] >> 16),
+                                d16(row, pq[j] & 0xFFFFu) + (int32_t)(cc[j] & 0xFFFFu)), INF);
+  }
+}
+template <bool CONN>
+__device__ __forceinline__ int32_t out_v(int32_t cp, int32_t rp, int32_t cq, int32_t rq) {
+  return CONN ? __viaddmin_s32(cq, rq, cp + rp) : out_val(cp, rp, cq, rq);
 }
 
+template <bool CONN>
 __global__ void __launch_bounds__(XP_NT, 1)
     k_expand_pairs(const uint16_t *__restrict__ D16, int32_t ldr, int32_t nr, const VDesc *__restrict__ desc,
                    const XpView X, int32_t n, int32_t rb, int32_t re, int32_t *__restrict__ out, int64_t ldo,
                    int32_t gcap, int32_t *counter) {
   extern __shared__ __align__(16) uint16_t srow[];   // [1 + gcap][ldr]
   __shared__ int4 meta[XP_RMAX];                     // {c_sv, c_sx, slot, local output row}
+  __shared__ int4 runs[XP_RMAX];                     // {slot, first meta row, end}: one per pair in the sweep
   __shared__ int32_t slot_x[XP_GMAX];
-  __shared__ int32_t s_item, s_nrow, s_ns, s_pj, s_rj;
+  __shared__ int32_t s_item, s_nrow, s_ns, s_pj, s_rj, s_nrun;
   const int tid = threadIdx.x;
   const uint32_t ldo_b = (uint32_t)(ldo * 4);
   for (;;) {
@@ -393,7 +408,7 @@ __global__ void __launch_bounds__(XP_NT, 1)
     for (;;) {
       if (tid < 32) {   // warp 0 builds the next sweep: up to gcap partner rows, XP_RMAX chain rows in range
         const int lane = tid;
-        int ns = 0, nrow = 0;   // warp-uniform
+        int ns = 0, nrow = 0, nrun = 0;   // warp-uniform
         while (pj < pe && nrow < XP_RMAX) {
           const int32_t x = X.px[pj];
           int slot = 0;
@@ -409,6 +424,7 @@ __global__ void __launch_bounds__(XP_NT, 1)
             }
           }
           const int32_t r1 = X.pstart[pj + 1];
+          const int m0 = nrow;
           while (rj < r1 && nrow < XP_RMAX) {   // 32 rows of the pair at a time
             const int32_t idx = rj + lane;
             bool in = false;
@@ -436,16 +452,20 @@ __global__ void __launch_bounds__(XP_NT, 1)
               nrow = XP_RMAX;
             }
           }
+          if (nrow > m0) {
+            if (lane == 0) runs[nrun] = make_int4(slot, m0, nrow, 0);
+            ++nrun;
+          }
           if (rj >= r1) {
             ++pj;
             if (pj < pe) rj = X.pstart[pj];
           }
         }
         __syncwarp();
-        if (lane == 0) { s_nrow = nrow; s_ns = ns; s_pj = pj; s_rj = rj; }
+        if (lane == 0) { s_nrow = nrow; s_ns = ns; s_pj = pj; s_rj = rj; s_nrun = nrun; }
       }
       __syncthreads();
-      const int nrow = s_nrow, ns = s_ns;
+      const int nrow = s_nrow, ns = s_ns, nrun = s_nrun;
       pj = s_pj;
       rj = s_rj;
       if (nrow > 0 || need_term) {
@@ -459,12 +479,17 @@ __global__ void __launch_bounds__(XP_NT, 1)
                 reinterpret_cast<const uint4 *>(D16 + (int64_t)slot_x[k] * ldr)[i];
         loaded_v = true;
         __syncthreads();
+        // descriptors of the next column group are loaded while the current one is computed and stored
+        uint4 na = make_uint4(0, 0, 0, 0), nb4 = make_uint4(0, 0, 0, 0);
+        if (tid * 4 + 4 <= n) {
+          na = *reinterpret_cast<const uint4 *>(X.pd + tid * 4);
+          nb4 = *reinterpret_cast<const uint4 *>(X.pd + tid * 4 + 2);
+        }
         for (int32_t c0 = tid * 4; c0 < n; c0 += XP_NT * 4) {
           uint32_t pq[4], cc[4];
-          if (c0 + 4 <= n) {
-            const uint4 a = *reinterpret_cast<const uint4 *>(X.pd + c0);
-            const uint4 b = *reinterpret_cast<const uint4 *>(X.pd + c0 + 2);
-            pq[0] = a.x; cc[0] = a.y; pq[1] = a.z; cc[1] = a.w; pq[2] = b.x; cc[2] = b.y; pq[3] = b.z; cc[3] = b.w;
+          const bool full = c0 + 4 <= n;
+          if (full) {
+            pq[0] = na.x; cc[0] = na.y; pq[1] = na.z; cc[1] = na.w; pq[2] = nb4.x; cc[2] = nb4.y; pq[3] = nb4.z; cc[3] = nb4.w;
           } else {
 #pragma unroll
             for (int j = 0; j < 4; ++j) {
@@ -472,31 +497,40 @@ __global__ void __launch_bounds__(XP_NT, 1)
               pq[j] = q.x; cc[j] = q.y;
             }
           }
-          int32_t Rv[4], R1[4], R2[4], R3[4], R4[4];
-          r_of(srow, pq, cc, Rv);
-          if (ns > 0) r_of(srow + ldr, pq, cc, R1);
-          if (ns > 1) r_of(srow + 2 * ldr, pq, cc, R2);
-          if (ns > 2) r_of(srow + 3 * ldr, pq, cc, R3);
-          if (ns > 3) r_of(srow + 4 * ldr, pq, cc, R4);
-          const bool full = c0 + 4 <= n;
+          const int32_t c1 = c0 + XP_NT * 4;
+          if (c1 + 4 <= n) {
+            na = *reinterpret_cast<const uint4 *>(X.pd + c1);
+            nb4 = *reinterpret_cast<const uint4 *>(X.pd + c1 + 2);
+          }
+          int32_t Rv[4];
+          r_of<CONN>(srow, pq, cc, Rv);
           if (need_term) {
             int32_t *o = reinterpret_cast<int32_t *>(reinterpret_cast<char *>(out) + (uint64_t)(uint32_t)(tv - rb) * ldo_b) + c0;
             if (full) st_cs_v4(o, make_int4(Rv[0], Rv[1], Rv[2], Rv[3]));
             else for (int j = 0; c0 + j < n; ++j) o[j] = Rv[j];
           }
-          for (int r = 0; r < nrow; ++r) {
-            const int4 m = meta[r];
-            const int32_t *Rx = m.z == 0 ? Rv : m.z == 1 ? R1 : m.z == 2 ? R2 : m.z == 3 ? R3 : R4;
-            int4 o4;
-            o4.x = out_val(m.x, Rv[0], m.y, Rx[0]);
-            o4.y = out_val(m.x, Rv[1], m.y, Rx[1]);
-            o4.z = out_val(m.x, Rv[2], m.y, Rx[2]);
-            o4.w = out_val(m.x, Rv[3], m.y, Rx[3]);
-            int32_t *o = reinterpret_cast<int32_t *>(reinterpret_cast<char *>(out) + (uint64_t)(uint32_t)m.w * ldo_b) + c0;
-            if (full) st_cs_v4(o, o4);
-            else {
-              const int32_t t4[4] = {o4.x, o4.y, o4.z, o4.w};
-              for (int j = 0; c0 + j < n; ++j) o[j] = t4[j];
+          for (int ru = 0; ru < nrun; ++ru) {
+            const int4 R = runs[ru];
+            int32_t Rx[4];
+            if (R.x == 0) {
+#pragma unroll
+              for (int j = 0; j < 4; ++j) Rx[j] = Rv[j];
+            } else {
+              r_of<CONN>(srow + R.x * ldr, pq, cc, Rx);
+            }
+            for (int r = R.y; r < R.z; ++r) {
+              const int4 m = meta[r];
+              int4 o4;
+              o4.x = out_v<CONN>(m.x, Rv[0], m.y, Rx[0]);
+              o4.y = out_v<CONN>(m.x, Rv[1], m.y, Rx[1]);
+              o4.z = out_v<CONN>(m.x, Rv[2], m.y, Rx[2]);
+              o4.w = out_v<CONN>(m.x, Rv[3], m.y, Rx[3]);
+              int32_t *o = reinterpret_cast<int32_t *>(reinterpret_cast<char *>(out) + (uint64_t)(uint32_t)m.w * ldo_b) + c0;
+              if (full) st_cs_v4(o, o4);
+              else {
+                const int32_t t4[4] = {o4.x, o4.y, o4.z, o4.w};
+                for (int j = 0; c0 + j < n; ++j) o[j] = t4[j];
+              }
             }
           }
         }
@@ -622,15 +656,20 @@ ear_status_t launch_pairs(const ear_plan_s *plan, const uint16_t *D16, int32_t l
   const ear_xp_s *x = plan->xp;
   const int32_t nr = plan->n_reduced, gcap = xp_gcap(nr);
   const int smem = (int)((1 + gcap) * (int64_t)ld16 * 2);
-  EAR_CUDA_TRY(smem_attr((const void *)k_expand_pairs, smem));
+  const bool conn = plan->connected == 1;
+  EAR_CUDA_TRY(smem_attr(conn ? (const void *)k_expand_pairs<true> : (const void *)k_expand_pairs<false>, smem));
   int32_t *counter = nullptr;
   EAR_CUDA_TRY(cudaMallocAsync((void **)&counter, sizeof(int32_t), st));
   EAR_CUDA_TRY(dev_memset(counter, 0, sizeof(int32_t), st));
   const XpView V{x->pd, x->rows, x->pstart, x->px, x->istart, x->tid2v};
   const double rows = row_end - row_begin;
   int se = prof_begin(prof_kind, st);
-  EAR_LAUNCH(k_expand_pairs, num_sms(), XP_NT, smem, st)(D16, ld16, nr, plan->desc, V, plan->n, row_begin, row_end, out,
-                                                        ldo, gcap, counter);
+  if (conn)
+    EAR_LAUNCH(k_expand_pairs<true>, num_sms(), XP_NT, smem, st)(D16, ld16, nr, plan->desc, V, plan->n, row_begin,
+                                                                  row_end, out, ldo, gcap, counter);
+  else
+    EAR_LAUNCH(k_expand_pairs<false>, num_sms(), XP_NT, smem, st)(D16, ld16, nr, plan->desc, V, plan->n, row_begin,
+                                                                   row_end, out, ldo, gcap, counter);
   // algorithmic bytes: the output, D read once (counted as the int32 D, as for the row-group kernel), the
   // descriptors
   prof_end(se, st, 4.0 * rows * plan->n + 16.0 * plan->n + 4.0 * (double)nr * nr * rows / plan->n);

@@ -890,7 +890,9 @@ ear_status_t part_prepare(ear_plan_s *p, cudaStream_t st) {
   }
   GView gv;
   EAR_TRY(plan_view(p, st, &gv));
-  return part_build(gv, st, &p->part);
+  EAR_TRY(part_build(gv, st, &p->part));
+  p->connected = p->part->multi ? 0 : 1;   // every region in one component <=> G^r connected
+  return EAR_OK;
 }
 
 // Every row of the view's distance matrix as u16 (0xFFFF = INF, row stride ldo >= round_up(n, 8)) into
