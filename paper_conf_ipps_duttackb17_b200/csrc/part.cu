@@ -38,6 +38,7 @@
 #include <cub/cub.cuh>
 
 #include <algorithm>
+#include <chrono>
 #include <climits>
 #include <cstdlib>
 
@@ -57,9 +58,7 @@ struct ear_part_s {
   int32_t *gidx = nullptr;           // [nr] global boundary index, -1 inside
   int32_t *big = nullptr;            // [nbig] regions with |B_i| > MP_KC (the general product kernel)
   int32_t nbig = 0;
-  int32_t *itemoff = nullptr;        // [K+1] first k_region_final item of region i (tiles of W_i columns)
-  int64_t items_ld = -1;             // the row length the item offsets were cut for
-  std::vector<int32_t> h_roff, h_bcnt;
+  int2 *vrange = nullptr;            // [K] smallest / largest vertex id of region i
 };
 
 namespace ear {
@@ -383,8 +382,9 @@ __global__ void __launch_bounds__(MP_NT)
                 const int32_t *__restrict__ boff, const int32_t *__restrict__ perm, const uint16_t *__restrict__ Bsrc,
                 int64_t ldb, int32_t ncols, uint16_t *__restrict__ out, int64_t ldo, const int32_t *__restrict__ reg,
                 const int32_t *__restrict__ loc, const int32_t *__restrict__ cc, const int32_t *__restrict__ rcomp,
-                int32_t multi, const int32_t *__restrict__ rlist) {
+                int32_t multi, const int32_t *__restrict__ rlist, const int32_t *__restrict__ stats) {
   __shared__ __align__(16) uint32_t As[MP_KC][PCAP];
+  if (stats[1] || stats[0] + stats[2] >= 0xFFFF || (FINAL && stats[0] + stats[3] >= 0xFFFF)) return;
   __shared__ __align__(16) uint16_t Bs[MP_KC][MP_BS];
   __shared__ int32_t cl[MP_TC], ccol[MP_TC];
   const int i = rlist ? rlist[blockIdx.y] : blockIdx.y, tid = threadIdx.x;
@@ -499,23 +499,34 @@ __device__ __forceinline__ void cp_async16(void *smem, const void *gmem, int byt
 __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::); }
 __device__ __forceinline__ void cp_async_wait1() { asm volatile("cp.async.wait_group 1;\n" ::: "memory"); }
 
-// (1) for the regions with |B_i| <= MP_KC, persistent.  The tile of region i is its r_i rows x W_i
-// columns, W_i = 16 * min(32, 256 / ceil(r_i / 8)) (every thread busy whatever the region size: thread
-// (ro, cg) owns rows ro*8..+8 and columns cg*16..+16); a CTA walks a contiguous range of (region, tile)
-// items in region-major order, so A = d_i(., B_i) is staged once per region, and the B rows (DBV rows of
-// B_i, contiguous in v) of the next tile stream into the other half of a double buffer by cp.async while
-// the current tile is computed.  Tiles without a vertex of the region skip the local-term checks.
+// The two products for the regions with |B_i| <= MP_KC, persistent.
+//   FINAL = false, (2): DBVt[v][g] = min_b d_i(v, b) + dB16[boff_i + b][g]   (B rows: dB16, row-major in g)
+//   FINAL = true,  (1): D16[u][v]  = min([v in R_i] d_i(u, v), min_b d_i(u, b) + DBV[boff_i + b][v]), INF
+//                       across components
+// The tile of region i is its r_i rows x W_i columns, W_i = 16 * min(32, 256 / ceil(r_i / 8)) (every
+// thread busy whatever the region size: thread (ro, cg) owns rows ro*8..+8 and columns cg*16..+16); a CTA
+// walks a contiguous range of (region, tile) items in region-major order, so A = d_i(., B_i) is staged
+// once per region, and the B rows of the next tile stream into the other half of a double buffer by
+// cp.async while the current tile is computed.  Only tiles that meet the region's vertex-id range look
+// for local columns.  Guard (uniform): nothing runs unless the u16 sums of this product cannot wrap,
+// stats[0] (Lmax) + stats[2] (max of dB) < 0xFFFF, for FINAL also stats[0] + stats[3] (max of DBV) <
+// 0xFFFF, and no region overflowed.
 constexpr int FW_MAXW = 512, FW_BS = FW_MAXW + 8;
+__device__ __forceinline__ int width_of(int32_t r) { return 16 * min(32, MP_NT / max(1, (r + 7) >> 3)); }
+
+template <bool FINAL>
 __global__ void __launch_bounds__(MP_NT, 2)
-    k_region_final(const uint16_t *__restrict__ LR, const int32_t *__restrict__ roff, const int32_t *__restrict__ bcnt,
-                   const int32_t *__restrict__ boff, const int32_t *__restrict__ perm,
-                   const uint16_t *__restrict__ DBV, int64_t ldv, int32_t n, uint16_t *__restrict__ out, int64_t ldo,
-                   const int32_t *__restrict__ reg, const int32_t *__restrict__ loc, const int32_t *__restrict__ cc,
-                   const int32_t *__restrict__ rcomp, int32_t multi, const int32_t *__restrict__ itemoff, int32_t K) {
+    k_region_prod(const uint16_t *__restrict__ LR, const int32_t *__restrict__ roff, const int32_t *__restrict__ bcnt,
+                  const int32_t *__restrict__ boff, const int32_t *__restrict__ perm,
+                  const uint16_t *__restrict__ Bsrc, int64_t ldb, int32_t ncols, uint16_t *__restrict__ out,
+                  int64_t ldo, const int32_t *__restrict__ reg, const int32_t *__restrict__ loc,
+                  const int32_t *__restrict__ cc, const int32_t *__restrict__ rcomp, const int2 *__restrict__ vrange,
+                  int32_t multi, const int32_t *__restrict__ itemoff, int32_t K, const int32_t *__restrict__ stats) {
   extern __shared__ __align__(16) uint8_t smraw[];
   uint32_t(*As)[PCAP] = reinterpret_cast<uint32_t(*)[PCAP]>(smraw);                                // [MP_KC][PCAP]
   uint16_t(*Bs)[MP_KC][FW_BS] = reinterpret_cast<uint16_t(*)[MP_KC][FW_BS]>(smraw + MP_KC * PCAP * 4);  // [2]
-  __shared__ int32_t cl[FW_MAXW], ccol[FW_MAXW];
+  __shared__ int32_t cl[FINAL ? FW_MAXW : 1], ccol[FINAL ? FW_MAXW : 1];
+  if (stats[1] || stats[0] + stats[2] >= 0xFFFF || (FINAL && stats[0] + stats[3] >= 0xFFFF)) return;
   const int tid = threadIdx.x;
   const int32_t total = itemoff[K];
   const int32_t t0 = (int32_t)((int64_t)total * blockIdx.x / gridDim.x);
@@ -531,56 +542,73 @@ __global__ void __launch_bounds__(MP_NT, 2)
     }
     ri = lo;
   }
-  auto width_of = [&](int32_t r) { return 16 * min(32, MP_NT / max(1, (r + 7) >> 3)); };
-  auto issue = [&](int32_t t, int i, int buf) {
-    const int32_t r = roff[i + 1] - roff[i], nb = bcnt[i], b0 = boff[i];
-    const int32_t W = width_of(r), c0 = (t - itemoff[i]) * W;
+  // the next tile's B rows: region i, tile t (every thread issues its share of the 16-byte chunks)
+  auto issue = [&](int32_t t, int i, int32_t nb, int32_t b0, int32_t W, int buf) {
+    const int32_t c0 = (t - itemoff[i]) * W;
     const int chunks = W / 8;
     for (int e = tid; e < nb * chunks; e += MP_NT) {
       const int k = e / chunks, c8 = (e % chunks) * 8;
-      const bool ok = c0 + c8 < ldv;
-      cp_async16(&Bs[buf][k][c8], DBV + (int64_t)(b0 + k) * ldv + (ok ? c0 + c8 : 0), ok ? 16 : 0);
+      const bool ok = c0 + c8 < ldb;
+      cp_async16(&Bs[buf][k][c8], Bsrc + (int64_t)(b0 + k) * ldb + (ok ? c0 + c8 : 0), ok ? 16 : 0);
     }
     cp_async_commit();
   };
+  __shared__ int32_t s_perm[PCAP];
   int cur = -1, buf = 0;
-  issue(t0, ri, 0);
+  int32_t r0 = 0, r = 0, nb = 0, b0 = 0, W = 16, cgs = 1, nro = 0, cgi = 0, ro = 0, i_off = 0;
+  int2 vr = make_int2(0, -1);
+  {
+    const int32_t rr = roff[ri + 1] - roff[ri];
+    issue(t0, ri, bcnt[ri], boff[ri], width_of(rr), 0);
+  }
   for (int32_t t = t0; t < t1; ++t) {
     while (itemoff[ri + 1] <= t) ++ri;
     const int i = ri;
-    const int32_t r0 = roff[i], r = roff[i + 1] - r0, nb = bcnt[i];
-    const int32_t nro = (r + 7) >> 3, W = width_of(r), cgs = W / 16, c0 = (t - itemoff[i]) * W;
-    __syncthreads();   // tile t-1 is done with As, Bs[buf ^ 1], cl
-    if (i != cur) {
+    __syncthreads();   // tile t-1 is done with As, Bs[buf ^ 1], cl, s_perm
+    if (i != cur) {    // per-region constants and staging: A, the member ids
       cur = i;
+      r0 = roff[i], r = roff[i + 1] - r0, nb = bcnt[i], b0 = boff[i];
+      nro = (r + 7) >> 3, W = width_of(r), cgs = W / 16, cgi = tid % cgs, ro = tid / cgs;
+      i_off = itemoff[i];
+      if (FINAL) vr = vrange[i];
       const uint16_t *L = LR + (size_t)i * PCAP * PCAP;
       for (int e = tid; e < nb * PCAP; e += MP_NT) {
         const int k = e / PCAP, u = e % PCAP;
         As[k][u] = u < r ? dup16(L[k * PCAP + u]) : 0xFFFFFFFFu;
       }
+      for (int u = tid; u < r; u += MP_NT) s_perm[u] = perm[r0 + u];
     }
+    const int32_t c0 = (t - i_off) * W;
     int loc_any = 0;
-    for (int c = tid; c < W; c += MP_NT) {
-      const int32_t v = c0 + c;
-      int32_t lc = -1, cv = 0;
-      if (v < n) {
-        if (reg[v] == i) lc = loc[v];
-        if (multi) cv = cc[v];
+    if (FINAL) {
+      const bool meets = c0 <= vr.y && c0 + W > vr.x;
+      if (meets || multi) {
+        for (int c = tid; c < W; c += MP_NT) {
+          const int32_t v = c0 + c;
+          int32_t lc = -1, cv = 0;
+          if (v < ncols) {
+            if (meets && reg[v] == i) lc = loc[v];
+            if (multi) cv = cc[v];
+          }
+          cl[c] = lc;
+          ccol[c] = cv;
+          loc_any |= lc >= 0;
+        }
       }
-      cl[c] = lc;
-      ccol[c] = cv;
-      loc_any |= lc >= 0;
     }
     if (t + 1 < t1) {
-      int in = ri;
-      while (itemoff[in + 1] <= t + 1) ++in;
-      issue(t + 1, in, buf ^ 1);
+      if (itemoff[i + 1] > t + 1) {
+        issue(t + 1, i, nb, b0, W, buf ^ 1);
+      } else {
+        int in = i + 1;
+        while (itemoff[in + 1] <= t + 1) ++in;
+        issue(t + 1, in, bcnt[in], boff[in], width_of(roff[in + 1] - roff[in]), buf ^ 1);
+      }
     } else {
       cp_async_commit();   // keep the group count uniform
     }
     cp_async_wait1();
     loc_any = __syncthreads_or(loc_any);
-    const int cgi = tid % cgs, ro = tid / cgs;
     if (ro < nro) {
       uint32_t acc[8][8];
 #pragma unroll
@@ -601,8 +629,8 @@ __global__ void __launch_bounds__(MP_NT, 2)
           for (int p = 0; p < 8; ++p) acc[q][p] = __viaddmin_u16x2(a[q], b[p], acc[q][p]);
       }
       const uint16_t *L = LR + (size_t)i * PCAP * PCAP;
-      const int rc = multi ? rcomp[i] : 0;
-      const bool fix = loc_any || multi || c0 + W > n;
+      const int rc = FINAL && multi ? rcomp[i] : 0;
+      const bool fix = FINAL && (loc_any || multi || c0 + W > ncols);
       const int cb = c0 + cgi * 16;
 #pragma unroll
       for (int q = 0; q < 8; ++q) {
@@ -616,14 +644,16 @@ __global__ void __launch_bounds__(MP_NT, 2)
             for (int p = 0; p < 8; ++p) {
               uint32_t lo = o[p] & 0xFFFFu, hi = o[p] >> 16;
               const int ca = cgi * 16 + 2 * p;
-              if (cl[ca] >= 0) lo = min(lo, (uint32_t)L[u * PCAP + cl[ca]]);
-              if (cl[ca + 1] >= 0) hi = min(hi, (uint32_t)L[u * PCAP + cl[ca + 1]]);
-              if (c0 + ca >= n || (multi && ccol[ca] != rc)) lo = 0xFFFFu;
-              if (c0 + ca + 1 >= n || (multi && ccol[ca + 1] != rc)) hi = 0xFFFFu;
+              if (loc_any) {
+                if (cl[ca] >= 0) lo = min(lo, (uint32_t)L[u * PCAP + cl[ca]]);
+                if (cl[ca + 1] >= 0) hi = min(hi, (uint32_t)L[u * PCAP + cl[ca + 1]]);
+              }
+              if (c0 + ca >= ncols || (multi && ccol[ca] != rc)) lo = 0xFFFFu;
+              if (c0 + ca + 1 >= ncols || (multi && ccol[ca + 1] != rc)) hi = 0xFFFFu;
               o[p] = lo | (hi << 16);
             }
           }
-          uint16_t *dst = out + (int64_t)perm[r0 + u] * ldo + cb;
+          uint16_t *dst = out + (int64_t)s_perm[u] * ldo + cb;
           if (cb < ldo) *reinterpret_cast<uint4 *>(dst) = make_uint4(o[0], o[1], o[2], o[3]);
           if (cb + 8 < ldo) *reinterpret_cast<uint4 *>(dst + 8) = make_uint4(o[4], o[5], o[6], o[7]);
         }
@@ -632,6 +662,46 @@ __global__ void __launch_bounds__(MP_NT, 2)
     buf ^= 1;
   }
 }
+
+// item offsets of k_region_prod: region i contributes ceil(ncols / W_i) tiles (none when |B_i| > MP_KC:
+// the general kernel does it); one CTA, chunked block scan
+__global__ void __launch_bounds__(1024) k_items(const int32_t *__restrict__ roff, const int32_t *__restrict__ bcnt,
+                                                int32_t K, int32_t ncols, int32_t *itemoff) {
+  __shared__ int32_t part[1024];
+  __shared__ int32_t carry;
+  if (threadIdx.x == 0) carry = 0;
+  for (int base = 0; base < K; base += 1024) {
+    const int i = base + threadIdx.x;
+    int32_t c = 0;
+    if (i < K && bcnt[i] <= MP_KC) c = (ncols + width_of(roff[i + 1] - roff[i]) - 1) / width_of(roff[i + 1] - roff[i]);
+    part[threadIdx.x] = c;
+    __syncthreads();
+    for (int o = 1; o < 1024; o <<= 1) {   // inclusive Hillis-Steele scan
+      const int32_t x = threadIdx.x >= o ? part[threadIdx.x - o] : 0;
+      __syncthreads();
+      part[threadIdx.x] += x;
+      __syncthreads();
+    }
+    if (i < K) itemoff[i + 1] = carry + part[threadIdx.x];
+    __syncthreads();
+    if (threadIdx.x == 1023) carry += part[1023];
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) itemoff[0] = 0;
+}
+
+// smallest and largest vertex id of every region (k_region_prod's local-column test)
+__global__ void k_vrange(const int32_t *__restrict__ perm, const int32_t *__restrict__ roff, int32_t K, int2 *vr) {
+  for (int32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < K; i += gridDim.x * blockDim.x) {
+    int32_t lo = INT_MAX, hi = -1;
+    for (int32_t e = roff[i]; e < roff[i + 1]; ++e) {
+      lo = min(lo, perm[e]);
+      hi = max(hi, perm[e]);
+    }
+    vr[i] = make_int2(lo, hi);
+  }
+}
+
 constexpr int FINAL_SMEM = MP_KC * PCAP * 4 + 2 * MP_KC * FW_BS * 2;
 
 // The boundary graph H of a level: vertex g = global boundary index; arcs: the clique of its region's
@@ -688,18 +758,20 @@ __global__ void k_h_cc(const int32_t *__restrict__ bvert, const int32_t *__restr
   }
 }
 
-// largest entry < 0xFFFF of a u16 matrix (rows x ld, ld % 8 == 0)
-__global__ void k_max16(const uint16_t *__restrict__ M, int32_t rows, int64_t ld, int32_t *out) {
+// largest entry < 0xFFFF of the first `cols` columns of a u16 matrix (rows x ld, ld % 8 == 0)
+__global__ void k_max16(const uint16_t *__restrict__ M, int32_t rows, int64_t ld, int32_t cols, int32_t *out) {
   const int64_t tot = (int64_t)rows * (ld / 8);
   uint32_t mx = 0;
   for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < tot; e += (int64_t)gridDim.x * blockDim.x) {
+    const int32_t c8 = (int32_t)(e % (ld / 8)) * 8;
+    if (c8 >= cols) continue;
     const uint4 v = reinterpret_cast<const uint4 *>(M)[e];
     const uint32_t w4[4] = {v.x, v.y, v.z, v.w};
 #pragma unroll
     for (int j = 0; j < 4; ++j) {
       const uint32_t lo = w4[j] & 0xFFFFu, hi = w4[j] >> 16;
-      if (lo != 0xFFFFu) mx = max(mx, lo);
-      if (hi != 0xFFFFu) mx = max(mx, hi);
+      if (lo != 0xFFFFu && c8 + 2 * j < cols) mx = max(mx, lo);
+      if (hi != 0xFFFFu && c8 + 2 * j + 1 < cols) mx = max(mx, hi);
     }
   }
   for (int o = 16; o; o >>= 1) mx = max(mx, __shfl_xor_sync(0xffffffffu, mx, o));
@@ -722,6 +794,29 @@ __global__ void k_widen(const uint16_t *__restrict__ D16, int64_t ld16, int32_t 
     D[(int64_t)r * ldd + c] = x;
   }
 }
+
+// EAR_PART_TRACE=1 (lab): host time at stage boundaries, each synchronised
+struct Trace {
+  cudaStream_t st;
+  int depth;
+  bool on;
+  std::chrono::steady_clock::time_point t0;
+  Trace(cudaStream_t s, int d) : st(s), depth(d) {
+    static const bool env = getenv("EAR_PART_TRACE") != nullptr;
+    on = env;
+    if (on) {
+      cudaStreamSynchronize(st);
+      t0 = std::chrono::steady_clock::now();
+    }
+  }
+  void mark(const char *what) {
+    if (!on) return;
+    cudaStreamSynchronize(st);
+    const auto t = std::chrono::steady_clock::now();
+    fprintf(stderr, "[part d%d] %-22s %8.3f ms\n", depth, what, std::chrono::duration<double, std::milli>(t - t0).count());
+    t0 = t;
+  }
+};
 
 struct Tmp {
   cudaStream_t st;
@@ -753,7 +848,7 @@ ear_status_t rb1(void *h, const void *d, size_t bytes, cudaStream_t st, const ch
 
 void part_free(ear_part_s *q, cudaStream_t st) {
   if (!q) return;
-  void *a[] = {q->reg, q->loc, q->perm, q->roff, q->bcnt, q->boff, q->rcomp, q->bvert, q->gidx, q->big, q->itemoff};
+  void *a[] = {q->reg, q->loc, q->perm, q->roff, q->bcnt, q->boff, q->rcomp, q->bvert, q->gidx, q->big, q->vrange};
   for (void *x : a)
     if (x) cudaFreeAsync(x, st);
   delete q;
@@ -780,6 +875,7 @@ ear_status_t part_build(const GView &gv, cudaStream_t st, ear_part_s **out) {
     return s;
   };
   const int g = grid_n(n);
+  Trace tr(st, -1);
   EAR_LAUNCH(k_seed, g, NT, 0, st)(cc, n, PSEED, lab[0], grp);
   int cur = 0, passes = 0;
   for (int32_t S2 = PSEED / 2;; S2 = std::max(1, S2 / 2)) {
@@ -809,6 +905,7 @@ ear_status_t part_build(const GView &gv, cudaStream_t st, ear_part_s **out) {
     if (passes > 12) return fail((set_error("part_prepare: region splitting did not converge"), EAR_ECUDA));
   }
   q->passes = passes;
+  tr.mark("build: bfs+split");
   // members by (region, boundary first, id)
   EAR_LAUNCH(k_keys, g, NT, 0, st)(rowptr, col, n, lab[cur], keys, vals);
   if (cudaMallocAsync((void **)&q->perm, sizeof(int32_t) * n, st) != cudaSuccess)
@@ -841,6 +938,7 @@ ear_status_t part_build(const GView &gv, cudaStream_t st, ear_part_s **out) {
     ear_status_t s = rb1(h, flags, sizeof(h), st, "part_prepare");
     if (s != EAR_OK) return fail(s);
   }
+  tr.mark("build: sort+fill");
   q->K = h[0];
   q->NB = h[1];
   q->max_region = h[2];
@@ -853,8 +951,6 @@ ear_status_t part_build(const GView &gv, cudaStream_t st, ear_part_s **out) {
   EAR_CUDA_TRY(cudaStreamSynchronize(st));
   q->sum_rb = 0;
   q->max_bnd = 0;
-  q->h_roff = hro;
-  q->h_bcnt = hbc;
   std::vector<int32_t> big;
   for (int i = 0; i < q->K; ++i) {
     q->sum_rb += (double)(hro[i + 1] - hro[i]) * hbc[i];
@@ -869,6 +965,10 @@ ear_status_t part_build(const GView &gv, cudaStream_t st, ear_part_s **out) {
     EAR_CUDA_TRY(cudaMemcpyAsync(q->big, big.data(), sizeof(int32_t) * big.size(), cudaMemcpyHostToDevice, st));
     EAR_CUDA_TRY(cudaStreamSynchronize(st));
   }
+  if (cudaMallocAsync((void **)&q->vrange, sizeof(int2) * q->K, st) != cudaSuccess)
+    return fail((set_error("part_prepare: out of device memory"), EAR_ENOMEM));
+  EAR_LAUNCH(k_vrange, grid_n(q->K), NT, 0, st)(q->perm, q->roff, q->K, q->vrange);
+  tr.mark("build: host lists");
   *out = q;
   EAR_CUDA_TRY(cudaGetLastError());
   return EAR_OK;
@@ -906,6 +1006,7 @@ ear_status_t part_solve(const GView &gv, ear_part_s *q, uint16_t *out, int64_t l
   // mostly tiny components (K near n): the (column blocks x regions) product grid would dominate
   if (q->K > n / 16 && (double)q->K * ceil_div(n, MP_TC) > 65536.0) return EAR_OK;
   const int ps = depth == 0 ? prof_begin(PK_PART, st) : -1;
+  Trace tr(st, depth);
   Tmp t(st);
   uint16_t *LR = nullptr, *dB16 = nullptr, *DBVt = nullptr, *DBV = nullptr;
   int32_t *stats = nullptr;
@@ -920,6 +1021,9 @@ ear_status_t part_solve(const GView &gv, ear_part_s *q, uint16_t *out, int64_t l
   EAR_CUDA_TRY(smem_attr((const void *)k_region_fw, fw_smem));
   EAR_LAUNCH(k_region_fw, q->K, FW_NT, fw_smem, st)(gv.rowptr, gv.col, gv.w, q->roff, q->perm, q->reg, q->loc, LR,
                                                      stats);
+  if (tr.on) fprintf(stderr, "[part d%d] n=%d K=%d NB=%d max_bnd=%d sum_rb=%.0f passes=%d\n", depth, n, q->K, NB,
+                     q->max_bnd, q->sum_rb, q->passes);
+  tr.mark("region fw");
   // (3): distances between boundary vertices
   if (NB > 0) {
     bool done = false;
@@ -950,11 +1054,13 @@ ear_status_t part_solve(const GView &gv, ear_part_s *q, uint16_t *out, int64_t l
       EAR_LAUNCH(k_h_cc, grid_n(NB), NT, 0, st)(q->bvert, gv.cc, NB, mn, hcc);
       const GView hv{NB, hrow, hcol, hw, hcc};
       ear_part_s *qh = nullptr;
+      tr.mark("H build");
       EAR_TRY(part_build(hv, st, &qh));
       ear_status_t s = part_solve(hv, qh, dB16, NBp, depth + 1, fw32, &done, st);
       part_free(qh, st);
       EAR_TRY(s);
-      if (done) EAR_LAUNCH(k_max16, grid_n((int64_t)NB * NBp / 8), NT, 0, st)(dB16, NB, NBp, stats + 2);
+      tr.mark("H solved");
+      if (done) EAR_LAUNCH(k_max16, grid_n((int64_t)NB * NBp / 8), NT, 0, st)(dB16, NB, NBp, NB, stats + 2);
     }
     if (!done) {   // dense: blocked FW over the boundary matrix
       int32_t *dB = nullptr, *labB = nullptr;
@@ -969,54 +1075,57 @@ ear_status_t part_solve(const GView &gv, ear_part_s *q, uint16_t *out, int64_t l
       EAR_LAUNCH(k_bnd_lab, grid_n(NpB), NT, 0, st)(q->bvert, gv.cc, NB, NpB, labB);
       EAR_TRY(fw_single(dB, NpB, NpB, st, labB, NB, !fw32, nullptr));
       EAR_LAUNCH(k_bnd_narrow, grid_n((int64_t)NB * NBp / 2), NT, 0, st)(dB, NpB, NB, NBp, dB16, stats + 2);
+      tr.mark("dense boundary fw");
     }
   }
-  int32_t h[4];
-  EAR_TRY(rb1(h, stats, sizeof(h), st, "part_solve"));
-  const int64_t Lmax = h[0], Dmax = h[2];
+  // the products, each guarded on the device by its no-wrap condition (stats: Lmax, region overflow, max
+  // of dB, max of DBV); one readback at the end decides whether the route applied
   if (ps >= 0) prof_end(ps, st, 0);
-  if (h[1] || Dmax + 2 * Lmax >= 0xFFFF) return EAR_OK;
   const int32_t *cc = q->multi ? gv.cc : nullptr;
   const int pm = depth == 0 ? prof_begin(PK_PART_MP, st) : -1;
   const int64_t ldv = round_up(n, 8);
+  int32_t *items = nullptr;
+  if (!t.get(&items, (size_t)q->K + 1)) {
+    set_error("part_solve: out of device memory");
+    return EAR_ENOMEM;
+  }
+  EAR_CUDA_TRY(smem_attr((const void *)k_region_prod<false>, FINAL_SMEM));
+  EAR_CUDA_TRY(smem_attr((const void *)k_region_prod<true>, FINAL_SMEM));
   if (NB > 0) {
-    dim3 g1(NBp / MP_TC, q->K);
-    EAR_LAUNCH(k_region_mp<false>, g1, MP_NT, 0, st)(LR, q->roff, q->bcnt, q->boff, q->perm, dB16, NBp, NBp, DBVt, NBp,
-                                                      q->reg, q->loc, cc, q->rcomp, q->multi, nullptr);
+    EAR_LAUNCH(k_items, 1, 1024, 0, st)(q->roff, q->bcnt, q->K, NB, items);
+    EAR_LAUNCH(k_region_prod<false>, 2 * num_sms(), MP_NT, FINAL_SMEM, st)(LR, q->roff, q->bcnt, q->boff, q->perm, dB16,
+                                                                          NBp, NB, DBVt, NBp, q->reg, q->loc, cc,
+                                                                          q->rcomp, q->vrange, q->multi, items, q->K,
+                                                                          stats);
+    if (q->nbig > 0) {
+      dim3 g1(NBp / MP_TC, q->nbig);
+      EAR_LAUNCH(k_region_mp<false>, g1, MP_NT, 0, st)(LR, q->roff, q->bcnt, q->boff, q->perm, dB16, NBp, NBp, DBVt,
+                                                        NBp, q->reg, q->loc, cc, q->rcomp, q->multi, q->big, stats);
+    }
     if (!t.get(&DBV, (size_t)NB * ldv)) {
       set_error("part_solve: out of device memory");
       return EAR_ENOMEM;
     }
     dim3 gt((unsigned)ceil_div(NB, TR), (unsigned)ceil_div(n, TR));
     EAR_LAUNCH(k_transpose16, gt, NT, 0, st)(DBVt, NBp, n, NB, DBV, ldv);
+    EAR_LAUNCH(k_max16, grid_n((int64_t)NB * ldv / 8), NT, 0, st)(DBV, NB, ldv, n, stats + 3);
   }
-  if (q->items_ld != ldo) {   // tiles of W_i columns per region (regions with a big boundary: none)
-    std::vector<int32_t> off(q->K + 1, 0);
-    for (int i = 0; i < q->K; ++i) {
-      const int32_t r = q->h_roff[i + 1] - q->h_roff[i];
-      const int32_t W = 16 * std::min(32, MP_NT / std::max(1, (r + 7) >> 3));
-      off[i + 1] = off[i] + (q->h_bcnt[i] > MP_KC ? 0 : (int32_t)ceil_div(n, W));
-    }
-    if (!q->itemoff && cudaMallocAsync((void **)&q->itemoff, sizeof(int32_t) * (q->K + 1), st) != cudaSuccess) {
-      set_error("part_solve: out of device memory");
-      return EAR_ENOMEM;
-    }
-    EAR_CUDA_TRY(cudaMemcpyAsync(q->itemoff, off.data(), sizeof(int32_t) * (q->K + 1), cudaMemcpyHostToDevice, st));
-    EAR_CUDA_TRY(cudaStreamSynchronize(st));
-    q->items_ld = ldo;
-  }
-  EAR_CUDA_TRY(smem_attr((const void *)k_region_final, FINAL_SMEM));
-  EAR_LAUNCH(k_region_final, 2 * num_sms(), MP_NT, FINAL_SMEM, st)(LR, q->roff, q->bcnt, q->boff, q->perm, DBV, ldv, n,
-                                                                    out, ldo, q->reg, q->loc, cc, q->rcomp, q->multi,
-                                                                    q->itemoff, q->K);
+  tr.mark("product1+T");
+  EAR_LAUNCH(k_items, 1, 1024, 0, st)(q->roff, q->bcnt, q->K, n, items);
+  EAR_LAUNCH(k_region_prod<true>, 2 * num_sms(), MP_NT, FINAL_SMEM, st)(LR, q->roff, q->bcnt, q->boff, q->perm, DBV,
+                                                                       ldv, n, out, ldo, q->reg, q->loc, cc, q->rcomp,
+                                                                       q->vrange, q->multi, items, q->K, stats);
   if (q->nbig > 0) {
     dim3 g2((unsigned)ceil_div(ldo, MP_TC), q->nbig);
     EAR_LAUNCH(k_region_mp<true>, g2, MP_NT, 0, st)(LR, q->roff, q->bcnt, q->boff, q->perm, DBVt, NBp, n, out, ldo,
-                                                     q->reg, q->loc, cc, q->rcomp, q->multi, q->big);
+                                                     q->reg, q->loc, cc, q->rcomp, q->multi, q->big, stats);
   }
   if (pm >= 0) prof_end(pm, st, (double)n * q->sum_rb + (double)NB * q->sum_rb);
+  int32_t h[4];
+  EAR_TRY(rb1(h, stats, sizeof(h), st, "part_solve"));
+  tr.mark("final product");
   EAR_CUDA_TRY(cudaGetLastError());
-  *applied = true;
+  *applied = !h[1] && h[0] + h[2] < 0xFFFF && h[0] + h[3] < 0xFFFF;
   return EAR_OK;
 }
 
