@@ -15,9 +15,9 @@
 // d_i(b, b') (b, b' in B_i) and the arcs of G^r that join two regions:
 //     d(b, b') = FW over B                                                                     (3)
 // The kernels, in that order:
-//   * k_seed / k_bfs / k_split: regions = Voronoi cells of a multi-source hop BFS (seeds every PSEED
-//     ids plus one vertex per connected component, ties to the smaller seed id), cells larger than
-//     PCAP split again inside themselves with denser seeds -- label-independent up to the seed choice;
+//   * k_partition (one cooperative launch): regions = Voronoi cells of a multi-source hop BFS (seeds
+//     every PSEED ids plus one vertex per connected component, ties to the smaller seed id), cells larger
+//     than PCAP split again inside themselves with denser seeds -- label-independent up to the seeds;
 //   * CUB radix sort of (region, boundary-first) keys -> every region's members contiguous, its
 //     boundary first; region / boundary offsets by scans;
 //   * k_region_fw: d_i for every region, one CTA per region, the PCAP x PCAP matrix in registers (8 x 16
@@ -35,6 +35,7 @@
 // involve INF (0xFFFF, other components) wrap, but they only reach entries of pairs in different
 // components, which the last product overwrites with INF.  Otherwise *applied = false and the caller
 // runs another Phase II route.
+#include <cooperative_groups.h>
 #include <cub/cub.cuh>
 
 #include <algorithm>
@@ -85,66 +86,6 @@ constexpr int PREC_DEPTH = 2;       // ... down to this nesting depth (then by t
 int grid_n(int64_t n) { return (int)std::max<int64_t>(1, std::min<int64_t>(ceil_div(n, NT), 148 * 16)); }
 
 __device__ __forceinline__ uint32_t dup16(uint32_t x) { return x | (x << 16); }
-
-__global__ void k_seed(const int32_t *__restrict__ cc, int32_t n, int32_t S, int32_t *lab, int32_t *grp) {
-  for (int32_t v = blockIdx.x * blockDim.x + threadIdx.x; v < n; v += gridDim.x * blockDim.x) {
-    lab[v] = (v % S == 0 || cc[v] == v) ? v : -1;
-    grp[v] = 0;
-  }
-}
-
-// one level of the multi-source BFS (Jacobi: an unlabelled vertex takes the smallest label among its
-// neighbours labelled in earlier levels, i.e. of its nearest seeds); only inside its group
-__global__ void k_bfs(const int32_t *__restrict__ rowptr, const int32_t *__restrict__ col, int32_t n,
-                      const int32_t *__restrict__ lin, int32_t *__restrict__ lout, const int32_t *__restrict__ grp,
-                      int32_t *changed) {
-  int ch = 0;
-  for (int32_t v = blockIdx.x * blockDim.x + threadIdx.x; v < n; v += gridDim.x * blockDim.x) {
-    int32_t l = lin[v];
-    if (l < 0) {
-      const int32_t g = grp[v];
-      int32_t m = INT_MAX;
-      for (int32_t a = rowptr[v], e = rowptr[v + 1]; a < e; ++a) {
-        const int32_t u = col[a];
-        const int32_t lu = lin[u];
-        if (lu >= 0 && grp[u] == g) m = min(m, lu);
-      }
-      if (m != INT_MAX) {
-        l = m;
-        ch = 1;
-      }
-    }
-    lout[v] = l;
-  }
-  if (__syncthreads_or(ch) && threadIdx.x == 0) *changed = 1;
-}
-
-__global__ void k_count(const int32_t *__restrict__ lab, int32_t n, int32_t *cnt, int32_t *bad) {
-  for (int32_t v = blockIdx.x * blockDim.x + threadIdx.x; v < n; v += gridDim.x * blockDim.x) {
-    const int32_t l = lab[v];
-    if (l < 0) {
-      *bad = 1;
-      continue;
-    }
-    atomicAdd(&cnt[l], 1);
-  }
-}
-
-// regions above PCAP: their members are unlabelled again except the denser seeds (the old seed and the
-// ids divisible by S2), and grouped by the old region so that the next BFS stays inside it
-__global__ void k_split(int32_t n, int32_t *lab, const int32_t *__restrict__ cnt, int32_t S2, int32_t *grp,
-                        int32_t *over) {
-  int o = 0;
-  for (int32_t v = blockIdx.x * blockDim.x + threadIdx.x; v < n; v += gridDim.x * blockDim.x) {
-    const int32_t l = lab[v];
-    grp[v] = l;
-    if (cnt[l] > PCAP) {
-      lab[v] = (v == l || v % S2 == 0) ? v : -1;
-      o = 1;
-    }
-  }
-  if (__syncthreads_or(o) && threadIdx.x == 0) *over = 1;
-}
 
 __global__ void k_keys(const int32_t *__restrict__ rowptr, const int32_t *__restrict__ col, int32_t n,
                        const int32_t *__restrict__ lab, uint32_t *keys, int32_t *vals) {
@@ -663,6 +604,8 @@ __global__ void __launch_bounds__(MP_NT, 2)
   }
 }
 
+constexpr int FINAL_SMEM = MP_KC * PCAP * 4 + 2 * MP_KC * FW_BS * 2;
+
 // item offsets of k_region_prod: region i contributes ceil(ncols / W_i) tiles (none when |B_i| > MP_KC:
 // the general kernel does it); one CTA, chunked block scan
 __global__ void __launch_bounds__(1024) k_items(const int32_t *__restrict__ roff, const int32_t *__restrict__ bcnt,
@@ -689,20 +632,6 @@ __global__ void __launch_bounds__(1024) k_items(const int32_t *__restrict__ roff
   }
   if (threadIdx.x == 0) itemoff[0] = 0;
 }
-
-// smallest and largest vertex id of every region (k_region_prod's local-column test)
-__global__ void k_vrange(const int32_t *__restrict__ perm, const int32_t *__restrict__ roff, int32_t K, int2 *vr) {
-  for (int32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < K; i += gridDim.x * blockDim.x) {
-    int32_t lo = INT_MAX, hi = -1;
-    for (int32_t e = roff[i]; e < roff[i + 1]; ++e) {
-      lo = min(lo, perm[e]);
-      hi = max(hi, perm[e]);
-    }
-    vr[i] = make_int2(lo, hi);
-  }
-}
-
-constexpr int FINAL_SMEM = MP_KC * PCAP * 4 + 2 * MP_KC * FW_BS * 2;
 
 // The boundary graph H of a level: vertex g = global boundary index; arcs: the clique of its region's
 // boundary with weights d_i (local indices: the boundary comes first in a region) and its joining arcs.
@@ -776,6 +705,112 @@ __global__ void k_max16(const uint16_t *__restrict__ M, int32_t rows, int64_t ld
   }
   for (int o = 16; o; o >>= 1) mx = max(mx, __shfl_xor_sync(0xffffffffu, mx, o));
   if ((threadIdx.x & 31) == 0 && mx) atomicMax(out, (int32_t)mx);
+}
+
+// All of the region labelling in one cooperative launch (grid-wide barriers between BFS levels): seeds,
+// Jacobi BFS levels until nothing changes, then -- while a cell exceeds PCAP -- counts, the denser
+// seeds of the oversized cells and BFS again inside them.  The final labels end in lab0.
+// st[0]: an unlabelled vertex remained; st[1]: passes; st[2]: did not converge; st[4..6]: level flags
+__global__ void __launch_bounds__(NT) k_partition(const int32_t *__restrict__ rowptr, const int32_t *__restrict__ col,
+                                                  const int32_t *__restrict__ cc, int32_t n, int32_t S, int32_t *lab0,
+                                                  int32_t *lab1, int32_t *grp, int32_t *cnt, int32_t *st) {
+  namespace cg = cooperative_groups;
+  cg::grid_group grid = cg::this_grid();
+  const int32_t tid0 = blockIdx.x * blockDim.x + threadIdx.x, stride = gridDim.x * blockDim.x;
+  for (int32_t v = tid0; v < n; v += stride) {
+    lab0[v] = (v % S == 0 || cc[v] == v) ? v : -1;
+    grp[v] = 0;
+  }
+  if (tid0 == 0) st[4] = st[5] = st[6] = 0;
+  grid.sync();
+  int32_t *lin = lab0, *lout = lab1;
+  int32_t S2 = max(1, S / 2);
+  int level = 0;
+  for (int pass = 1;; ++pass) {
+    for (;; ++level) {
+      const int f = level % 3;
+      int ch = 0;
+      for (int32_t v = tid0; v < n; v += stride) {
+        int32_t l = lin[v];
+        if (l < 0) {
+          const int32_t g = grp[v];
+          int32_t m = INT_MAX;
+          for (int32_t a = rowptr[v], e = rowptr[v + 1]; a < e; ++a) {
+            const int32_t u = col[a];
+            const int32_t lu = lin[u];
+            if (lu >= 0 && grp[u] == g) m = min(m, lu);
+          }
+          if (m != INT_MAX) {
+            l = m;
+            ch = 1;
+          }
+        }
+        lout[v] = l;
+      }
+      if (__syncthreads_or(ch) && threadIdx.x == 0) st[4 + f] = 1;
+      if (tid0 == 0) st[4 + (level + 1) % 3] = 0;   // read two levels ago, before the last barrier
+      grid.sync();
+      int32_t *x = lin;
+      lin = lout;
+      lout = x;
+      if (!st[4 + f]) break;
+      if (level > 4 * n + 8) {
+        if (tid0 == 0) st[2] = 1;
+        break;
+      }
+    }
+    ++level;   // the flag of the level that ended the BFS is not reused before it is cleared
+    // cell sizes, then the oversized cells get denser seeds (grp = old cell: the next BFS stays inside)
+    for (int32_t v = tid0; v < n; v += stride) cnt[v] = 0;
+    if (tid0 == 0) st[7] = 0;
+    grid.sync();
+    for (int32_t v = tid0; v < n; v += stride) {
+      const int32_t l = lin[v];
+      if (l < 0) st[0] = 1;
+      else atomicAdd(&cnt[l], 1);
+    }
+    grid.sync();
+    int o = 0;
+    for (int32_t v = tid0; v < n; v += stride) {
+      const int32_t l = lin[v];
+      grp[v] = l;
+      if (l >= 0 && cnt[l] > PCAP) {
+        lin[v] = (v == l || v % S2 == 0) ? v : -1;
+        o = 1;
+      }
+    }
+    if (__syncthreads_or(o) && threadIdx.x == 0) st[7] = 1;
+    grid.sync();
+    if (!st[7] || st[2] || pass > 12) {
+      if (tid0 == 0) st[1] = pass;
+      if (lin != lab0)
+        for (int32_t v = tid0; v < n; v += stride) lab0[v] = lin[v];
+      if (pass > 12 && st[7] && tid0 == 0) st[2] = 1;
+      return;
+    }
+    S2 = max(1, S2 / 2);
+  }
+}
+
+// per-region statistics and lists on the device (K = tot[0]): max |B_i|, sum |R_i||B_i|, several
+// components, the regions with |B_i| > MP_KC, the vertex-id range of every region
+__global__ void k_region_stats(const int32_t *__restrict__ perm, const int32_t *__restrict__ roff,
+                               const int32_t *__restrict__ bcnt, const int32_t *__restrict__ rcomp, int32_t *tot,
+                               int32_t *big, int2 *vr) {
+  const int32_t K = tot[0];
+  for (int32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < K; i += gridDim.x * blockDim.x) {
+    const int32_t b = bcnt[i], r = roff[i + 1] - roff[i];
+    atomicMax(&tot[3], b);
+    atomicAdd(reinterpret_cast<unsigned long long *>(tot + 6), (unsigned long long)r * b);
+    if (rcomp[i] != rcomp[0]) tot[4] = 1;
+    if (b > MP_KC) big[atomicAdd(&tot[5], 1)] = i;
+    int32_t lo = INT_MAX, hi = -1;
+    for (int32_t e = roff[i]; e < roff[i + 1]; ++e) {
+      lo = min(lo, perm[e]);
+      hi = max(hi, perm[e]);
+    }
+    vr[i] = make_int2(lo, hi);
+  }
 }
 
 // int32 D (Np x Np, INF, padding isolated) from the u16 rows
@@ -862,7 +897,7 @@ ear_status_t part_build(const GView &gv, cudaStream_t st, ear_part_s **out) {
   Tmp t(st);
   int32_t *lab[2], *grp, *cnt, *flags, *rid, *gpos, *fstart, *fbnd, *vals;
   uint32_t *keys, *skeys;
-  constexpr int NFLAGS = 64;
+  constexpr int NFLAGS = 64;   // [0..15] labelling, [16..23] region totals
   if (!t.get(&lab[0], n) || !t.get(&lab[1], n) || !t.get(&grp, n) || !t.get(&cnt, n) || !t.get(&flags, NFLAGS) ||
       !t.get(&rid, n) || !t.get(&gpos, n) || !t.get(&fstart, n) || !t.get(&fbnd, n) || !t.get(&vals, n) ||
       !t.get(&keys, n) || !t.get(&skeys, n)) {
@@ -876,35 +911,18 @@ ear_status_t part_build(const GView &gv, cudaStream_t st, ear_part_s **out) {
   };
   const int g = grid_n(n);
   Trace tr(st, -1);
-  EAR_LAUNCH(k_seed, g, NT, 0, st)(cc, n, PSEED, lab[0], grp);
-  int cur = 0, passes = 0;
-  for (int32_t S2 = PSEED / 2;; S2 = std::max(1, S2 / 2)) {
-    // BFS levels in batches of 8 launches, one readback per batch
-    for (int it = 0;; it += 8) {
-      EAR_CUDA_TRY(dev_memset(flags, 0, 8 * sizeof(int32_t), st));
-      for (int b = 0; b < 8; ++b) {
-        EAR_LAUNCH(k_bfs, g, NT, 0, st)(rowptr, col, n, lab[cur], lab[cur ^ 1], grp, flags + b);
-        cur ^= 1;
-      }
-      int32_t h[8];
-      ear_status_t s = rb1(h, flags, sizeof(h), st, "part_prepare");
-      if (s != EAR_OK) return fail(s);
-      if (!h[7]) break;
-      if (it > 4 * n) return fail((set_error("part_prepare: BFS did not converge"), EAR_ECUDA));
-    }
-    ++passes;
-    EAR_CUDA_TRY(dev_memset(cnt, 0, sizeof(int32_t) * n, st));
-    EAR_CUDA_TRY(dev_memset(flags, 0, 2 * sizeof(int32_t), st));
-    EAR_LAUNCH(k_count, g, NT, 0, st)(lab[cur], n, cnt, flags);
-    EAR_LAUNCH(k_split, g, NT, 0, st)(n, lab[cur], cnt, S2, grp, flags + 1);
-    int32_t h[2];
-    ear_status_t s = rb1(h, flags, sizeof(h), st, "part_prepare");
-    if (s != EAR_OK) return fail(s);
-    if (h[0]) return fail((set_error("part_prepare: unlabelled vertex after the BFS"), EAR_ECUDA));
-    if (!h[1]) break;
-    if (passes > 12) return fail((set_error("part_prepare: region splitting did not converge"), EAR_ECUDA));
+  {
+    int per_sm = 0;
+    EAR_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_partition, NT, 0));
+    const int gc = (int)std::max<int64_t>(1, std::min<int64_t>(ceil_div(n, NT), (int64_t)per_sm * num_sms()));
+    EAR_CUDA_TRY(dev_memset(flags, 0, 16 * sizeof(int32_t), st));
+    int32_t S = PSEED;
+    void *args[] = {(void *)&rowptr, (void *)&col, (void *)&cc, (void *)&n, (void *)&S, (void *)&lab[0], (void *)&lab[1],
+                    (void *)&grp, (void *)&cnt, (void *)&flags};
+    count_launch();
+    EAR_CUDA_TRY(cudaLaunchCooperativeKernel((const void *)k_partition, gc, NT, args, 0, st));
   }
-  q->passes = passes;
+  const int cur = 0;
   tr.mark("build: bfs+split");
   // members by (region, boundary first, id)
   EAR_LAUNCH(k_keys, g, NT, 0, st)(rowptr, col, n, lab[cur], keys, vals);
@@ -928,46 +946,31 @@ ear_status_t part_build(const GView &gv, cudaStream_t st, ear_part_s **out) {
   if (need(&q->reg, n) || need(&q->loc, n) || need(&q->gidx, n) || need(&q->roff, (size_t)n + 1) ||
       need(&q->boff, n) || need(&q->bcnt, n) || need(&q->rcomp, n) || need(&q->bvert, n))
     return fail((set_error("part_prepare: out of device memory"), EAR_ENOMEM));
+  if (need(&q->big, n) || cudaMallocAsync((void **)&q->vrange, sizeof(int2) * n, st) != cudaSuccess)
+    return fail((set_error("part_prepare: out of device memory"), EAR_ENOMEM));
   EAR_CUDA_TRY(dev_memset(q->bcnt, 0, sizeof(int32_t) * n, st));
-  EAR_CUDA_TRY(dev_memset(flags, 0, 4 * sizeof(int32_t), st));
+  int32_t *tot = flags + 16;   // K, NB, max region, max |B_i|, multi, nbig, sum |R_i||B_i| (u64)
+  EAR_CUDA_TRY(dev_memset(tot, 0, 8 * sizeof(int32_t), st));
   EAR_LAUNCH(k_fill, g, NT, 0, st)(q->perm, fstart, fbnd, rid, gpos, cc, n, q->reg, q->gidx, q->roff, q->boff, q->bcnt,
-                                   q->rcomp, q->bvert, flags);
-  EAR_LAUNCH(k_loc, g, NT, 0, st)(q->perm, rid, q->roff, n, q->loc, flags + 2);
-  int32_t h[4];
+                                   q->rcomp, q->bvert, tot);
+  EAR_LAUNCH(k_loc, g, NT, 0, st)(q->perm, rid, q->roff, n, q->loc, tot + 2);
+  EAR_LAUNCH(k_region_stats, g, NT, 0, st)(q->perm, q->roff, q->bcnt, q->rcomp, tot, q->big, q->vrange);
+  int32_t h[24];
   {
     ear_status_t s = rb1(h, flags, sizeof(h), st, "part_prepare");
     if (s != EAR_OK) return fail(s);
   }
-  tr.mark("build: sort+fill");
-  q->K = h[0];
-  q->NB = h[1];
-  q->max_region = h[2];
+  if (h[0]) return fail((set_error("part_prepare: unlabelled vertex after the BFS"), EAR_ECUDA));
+  if (h[2]) return fail((set_error("part_prepare: region labelling did not converge"), EAR_ECUDA));
+  q->passes = h[1];
+  q->K = h[16];
+  q->NB = h[17];
+  q->max_region = h[18];
+  q->max_bnd = h[19];
+  q->multi = h[20];
+  q->nbig = h[21];
+  q->sum_rb = (double)((uint64_t)(uint32_t)h[22] | ((uint64_t)(uint32_t)h[23] << 32));
   q->NBp = (int32_t)round_up(std::max(q->NB, 1), MP_TC);
-  // host copies of the small per-region counts (statistics: max |B_i|, sum |R_i||B_i|, components)
-  std::vector<int32_t> hro(q->K + 1), hbc(q->K), hrc(q->K);
-  EAR_CUDA_TRY(cudaMemcpyAsync(hro.data(), q->roff, sizeof(int32_t) * (q->K + 1), cudaMemcpyDeviceToHost, st));
-  EAR_CUDA_TRY(cudaMemcpyAsync(hbc.data(), q->bcnt, sizeof(int32_t) * q->K, cudaMemcpyDeviceToHost, st));
-  EAR_CUDA_TRY(cudaMemcpyAsync(hrc.data(), q->rcomp, sizeof(int32_t) * q->K, cudaMemcpyDeviceToHost, st));
-  EAR_CUDA_TRY(cudaStreamSynchronize(st));
-  q->sum_rb = 0;
-  q->max_bnd = 0;
-  std::vector<int32_t> big;
-  for (int i = 0; i < q->K; ++i) {
-    q->sum_rb += (double)(hro[i + 1] - hro[i]) * hbc[i];
-    q->max_bnd = std::max(q->max_bnd, hbc[i]);
-    if (hrc[i] != hrc[0]) q->multi = 1;
-    if (hbc[i] > MP_KC) big.push_back(i);
-  }
-  q->nbig = (int32_t)big.size();
-  if (!big.empty()) {
-    if (cudaMallocAsync((void **)&q->big, sizeof(int32_t) * big.size(), st) != cudaSuccess)
-      return fail((set_error("part_prepare: out of device memory"), EAR_ENOMEM));
-    EAR_CUDA_TRY(cudaMemcpyAsync(q->big, big.data(), sizeof(int32_t) * big.size(), cudaMemcpyHostToDevice, st));
-    EAR_CUDA_TRY(cudaStreamSynchronize(st));
-  }
-  if (cudaMallocAsync((void **)&q->vrange, sizeof(int2) * q->K, st) != cudaSuccess)
-    return fail((set_error("part_prepare: out of device memory"), EAR_ENOMEM));
-  EAR_LAUNCH(k_vrange, grid_n(q->K), NT, 0, st)(q->perm, q->roff, q->K, q->vrange);
   tr.mark("build: host lists");
   *out = q;
   EAR_CUDA_TRY(cudaGetLastError());
