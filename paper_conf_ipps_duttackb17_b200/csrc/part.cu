@@ -80,8 +80,9 @@ constexpr uint32_t PC16 = 0x7FFF;    // cap of the region FW (two capped values 
 constexpr int FW_NT = 512;
 constexpr int MP_NT = 256, MP_TC = 128, MP_KC = 32, MP_BS = MP_TC + 8;   // Bs row stride (u16): 4-way max
 constexpr int NT = 256;
-constexpr int PREC_MIN = 1024;      // a boundary graph this large is solved by regions again
+constexpr int PREC_MIN = 2048;      // a boundary graph this large is solved by regions again
 constexpr int PREC_DEPTH = 2;       // ... down to this nesting depth (then by the blocked FW)
+constexpr int FW64_MAX = 8192;      // dense boundary matrices up to this size: the 64-tile cooperative FW
 
 int grid_n(int64_t n) { return (int)std::max<int64_t>(1, std::min<int64_t>(ceil_div(n, NT), 148 * 16)); }
 
@@ -813,6 +814,181 @@ __global__ void k_region_stats(const int32_t *__restrict__ perm, const int32_t *
   }
 }
 
+// ----------------------------------------------------------------------------------------------
+// Dense FW on a small boundary matrix (|B| up to a few thousand) with 64 x 64 tiles, packed u16x2 capped
+// at PC16 (the argument of sec. 6a: exact below the cap), the whole schedule in one cooperative launch:
+// per round k, block 0 closes the pivot tile (64 barriers in shared memory), every block then takes
+// pivot-row tiles (k, j) -- written with their transposes (j, k), D stays symmetric -- and then upper
+// tiles (i <= j) of the rest, each written with its mirror; grid barriers between the three phases.
+// 128-row tiles (the TMA kernel of sec. 6a) leave this size latency bound: a round costs its serial
+// 128-step phase 1 and two tile-deep launches (~85 us at |B| ~ 1,000).
+constexpr int F64 = 64;
+__device__ __forceinline__ void f64_load(uint16_t (*dst)[F64], const uint16_t *M, int64_t ld, int ti, int tj) {
+  for (int e = threadIdx.x; e < F64 * F64 / 8; e += blockDim.x) {
+    const int r = e / 8, c8 = (e % 8) * 8;
+    *reinterpret_cast<uint4 *>(&dst[r][c8]) =
+        *reinterpret_cast<const uint4 *>(M + (int64_t)(ti * F64 + r) * ld + tj * F64 + c8);
+  }
+}
+// C (4 rows x 4 columns per thread) = min(C, A^T (x) B): A[m][r] (row m of the pivot-row tile of i), B[m][c]
+__device__ __forceinline__ void f64_mp(const uint16_t (*A)[F64], const uint16_t (*B)[F64], uint32_t c[4][2]) {
+  const int tr = threadIdx.x / 16, tc = threadIdx.x % 16;
+#pragma unroll 8
+  for (int m = 0; m < F64; ++m) {
+    const uint2 av = *reinterpret_cast<const uint2 *>(&A[m][tr * 4]);
+    const uint2 bv = *reinterpret_cast<const uint2 *>(&B[m][tc * 4]);
+    const uint32_t a[4] = {dup16(av.x & 0xFFFFu), dup16(av.x >> 16), dup16(av.y & 0xFFFFu), dup16(av.y >> 16)};
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      c[q][0] = __viaddmin_u16x2(a[q], bv.x, c[q][0]);
+      c[q][1] = __viaddmin_u16x2(a[q], bv.y, c[q][1]);
+    }
+  }
+}
+// write the thread's 4 x 4 block into tile (ti, tj) and -- mirror -- its transpose into (tj, ti)
+__device__ __forceinline__ void f64_store(uint16_t *M, int64_t ld, int ti, int tj, const uint32_t c[4][2], bool mirror) {
+  const int tr = threadIdx.x / 16, tc = threadIdx.x % 16;
+#pragma unroll
+  for (int q = 0; q < 4; ++q)
+    *reinterpret_cast<uint2 *>(M + (int64_t)(ti * F64 + tr * 4 + q) * ld + tj * F64 + tc * 4) = make_uint2(c[q][0], c[q][1]);
+  if (mirror) {
+#pragma unroll
+    for (int cc = 0; cc < 4; ++cc) {   // column tc*4+cc of the block = row of the transpose
+      const uint32_t lo = (c[0][cc >> 1] >> (16 * (cc & 1))) & 0xFFFFu, l1 = (c[1][cc >> 1] >> (16 * (cc & 1))) & 0xFFFFu;
+      const uint32_t l2 = (c[2][cc >> 1] >> (16 * (cc & 1))) & 0xFFFFu, l3 = (c[3][cc >> 1] >> (16 * (cc & 1))) & 0xFFFFu;
+      *reinterpret_cast<uint2 *>(M + (int64_t)(tj * F64 + tc * 4 + cc) * ld + ti * F64 + tr * 4) =
+          make_uint2(lo | (l1 << 16), l2 | (l3 << 16));
+    }
+  }
+}
+__global__ void __launch_bounds__(256) k_fw64(uint16_t *M, int32_t N) {
+  namespace cg = cooperative_groups;
+  cg::grid_group grid = cg::this_grid();
+  __shared__ __align__(16) uint16_t As[F64][F64], Bs[F64][F64];
+  const int T = N / F64, tid = threadIdx.x, tr = tid / 16, tc = tid % 16;
+  // phase 1 by block 0 (in shared memory, one barrier per step: an in-place step kk only reads row and
+  // column kk, which it does not change)
+  auto close_pivot = [&](int k) {
+    f64_load(As, M, N, k, k);
+    __syncthreads();
+    for (int kk = 0; kk < F64; ++kk) {
+      const uint2 bv = *reinterpret_cast<const uint2 *>(&As[kk][tc * 4]);
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        const uint32_t a = dup16(As[tr * 4 + q][kk]);
+        uint2 cv = *reinterpret_cast<const uint2 *>(&As[tr * 4 + q][tc * 4]);
+        cv.x = __viaddmin_u16x2(a, bv.x, cv.x);
+        cv.y = __viaddmin_u16x2(a, bv.y, cv.y);
+        *reinterpret_cast<uint2 *>(&As[tr * 4 + q][tc * 4]) = cv;
+      }
+      __syncthreads();
+    }
+  };
+  for (int k = 0; k < T; ++k) {
+    if (blockIdx.x == 0) {
+      close_pivot(k);
+#pragma unroll
+      for (int q = 0; q < 4; ++q)
+        *reinterpret_cast<uint2 *>(M + (int64_t)(k * F64 + tr * 4 + q) * N + k * F64 + tc * 4) =
+            *reinterpret_cast<const uint2 *>(&As[tr * 4 + q][tc * 4]);
+    }
+    grid.sync();
+    if (blockIdx.x != 0 && blockIdx.x < T - 1) {
+      f64_load(As, M, N, k, k);   // the closed pivot tile
+      __syncthreads();
+    }
+    // phase 2: pivot-row tiles (k, j) = min(C, P (x) C); P is closed and symmetric, so A[m][r] = P[m][r]
+    for (int jt = blockIdx.x; jt < T - 1; jt += gridDim.x) {
+      const int j = jt < k ? jt : jt + 1;
+      __syncthreads();
+      f64_load(Bs, M, N, k, j);
+      __syncthreads();
+      uint32_t c[4][2];
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        const uint2 x = *reinterpret_cast<const uint2 *>(&Bs[tr * 4 + q][tc * 4]);
+        c[q][0] = x.x, c[q][1] = x.y;
+      }
+      f64_mp(As, Bs, c);
+      f64_store(M, N, k, j, c, true);
+    }
+    grid.sync();
+    // phase 3: upper tiles (i <= j) off row / column k: C = min(C, row(k,i)^T (x) row(k,j)), mirrored
+    const int64_t nt = (int64_t)T * (T + 1) / 2;
+    for (int64_t e = blockIdx.x; e < nt; e += gridDim.x) {
+      int i = (int)((sqrt(8.0 * (double)e + 1.0) - 1.0) / 2.0);   // e -> (j = row of the triangle, i <= j)
+      while ((int64_t)(i + 1) * (i + 2) / 2 <= e) ++i;
+      while ((int64_t)i * (i + 1) / 2 > e) --i;
+      const int jj = i, ii = (int)(e - (int64_t)i * (i + 1) / 2);
+      if (ii == k || jj == k) continue;
+      __syncthreads();
+      f64_load(As, M, N, k, ii);
+      f64_load(Bs, M, N, k, jj);
+      __syncthreads();
+      uint32_t c[4][2];
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        const uint2 x = *reinterpret_cast<const uint2 *>(M + (int64_t)(ii * F64 + tr * 4 + q) * N + jj * F64 + tc * 4);
+        c[q][0] = x.x, c[q][1] = x.y;
+      }
+      f64_mp(As, Bs, c);
+      f64_store(M, N, ii, jj, c, ii != jj);
+    }
+    grid.sync();
+  }
+}
+
+__global__ void k_b16_fill(uint16_t *M, int32_t N) {
+  const int64_t tot = (int64_t)N * N;
+  for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < tot; e += (int64_t)gridDim.x * blockDim.x)
+    M[e] = (e / N == e % N) ? 0 : (uint16_t)PC16;
+}
+__global__ void k_b16_clique(const uint16_t *__restrict__ LR, const int32_t *__restrict__ bcnt,
+                             const int32_t *__restrict__ boff, uint16_t *M, int32_t N) {
+  const int i = blockIdx.x;
+  const int nb = bcnt[i], b0 = boff[i];
+  const uint16_t *L = LR + (size_t)i * PCAP * PCAP;
+  for (int e = threadIdx.x; e < nb * nb; e += blockDim.x) {
+    const int a = e / nb, b = e % nb;
+    M[(int64_t)(b0 + a) * N + b0 + b] = (uint16_t)min((uint32_t)L[a * PCAP + b], PC16);
+  }
+}
+__global__ void k_b16_cross(const int32_t *__restrict__ rowptr, const int32_t *__restrict__ col,
+                            const int32_t *__restrict__ w, const int32_t *__restrict__ bvert, int32_t NB,
+                            const int32_t *__restrict__ reg, const int32_t *__restrict__ gidx, uint16_t *M, int32_t N) {
+  for (int32_t g = blockIdx.x * blockDim.x + threadIdx.x; g < NB; g += gridDim.x * blockDim.x) {
+    const int32_t v = bvert[g], rv = reg[v];
+    for (int32_t a = rowptr[v], e = rowptr[v + 1]; a < e; ++a) {
+      const int32_t x = col[a];
+      if (reg[x] != rv) M[(int64_t)g * N + gidx[x]] = (uint16_t)min(w[a], (int32_t)PC16);   // one arc per pair
+    }
+  }
+}
+// capped FW result -> dB16 (0xFFFF = INF), its largest finite entry; *bad when a connected pair reached the cap
+__global__ void k_b16_narrow(const uint16_t *__restrict__ M, int32_t N, const int32_t *__restrict__ bvert,
+                             const int32_t *__restrict__ cc, int32_t NB, int32_t NBp, uint16_t *dB16, int32_t *stats,
+                             int32_t *bad) {
+  const int64_t tot = (int64_t)NB * NBp;
+  int mx = 0, b = 0;
+  for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < tot; e += (int64_t)gridDim.x * blockDim.x) {
+    const int32_t g = (int32_t)(e / NBp), h = (int32_t)(e % NBp);
+    uint16_t y = 0xFFFF;
+    if (h < NB) {
+      const uint32_t x = M[(int64_t)g * N + h];
+      if (x < PC16) {
+        y = (uint16_t)x;
+        mx = max(mx, (int)x);
+      } else if (cc[bvert[g]] == cc[bvert[h]]) {
+        b = 1;
+      }
+    }
+    dB16[e] = y;
+  }
+  for (int o = 16; o; o >>= 1) mx = max(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+  if ((threadIdx.x & 31) == 0 && mx) atomicMax(stats, mx);
+  if (__syncthreads_or(b) && threadIdx.x == 0) *bad = 1;
+}
+
 // int32 D (Np x Np, INF, padding isolated) from the u16 rows
 __global__ void k_widen(const uint16_t *__restrict__ D16, int64_t ld16, int32_t nr, int32_t *D, int64_t ldd,
                         int32_t Np) {
@@ -1030,7 +1206,11 @@ ear_status_t part_solve(const GView &gv, ear_part_s *q, uint16_t *out, int64_t l
   // (3): distances between boundary vertices
   if (NB > 0) {
     bool done = false;
-    if (depth < PREC_DEPTH && NB >= PREC_MIN) {
+    static const int prec_min = [] {   // lab knob: EAR_PREC_MIN
+      const char *e = getenv("EAR_PREC_MIN");
+      return e ? atoi(e) : PREC_MIN;
+    }();
+    if (depth < PREC_DEPTH && NB >= prec_min) {
       // the boundary graph H (cliques d_i on every B_i + the joining arcs) by the same route
       Tmp th(st);
       int32_t *hdeg, *hrow, *hcol, *hw, *hcc, *mn;
@@ -1064,6 +1244,34 @@ ear_status_t part_solve(const GView &gv, ear_part_s *q, uint16_t *out, int64_t l
       EAR_TRY(s);
       tr.mark("H solved");
       if (done) EAR_LAUNCH(k_max16, grid_n((int64_t)NB * NBp / 8), NT, 0, st)(dB16, NB, NBp, NB, stats + 2);
+    }
+    if (!done && !fw32 && NB <= FW64_MAX) {   // dense, small: the cooperative 64-tile FW (capped u16)
+      uint16_t *M = nullptr;
+      int32_t *bad = nullptr;
+      const int32_t N64 = (int32_t)round_up(NB, F64);
+      if (!t.get(&M, (size_t)N64 * N64) || !t.get(&bad, 1)) {
+        set_error("part_solve: out of device memory");
+        return EAR_ENOMEM;
+      }
+      EAR_CUDA_TRY(dev_memset(bad, 0, sizeof(int32_t), st));
+      EAR_LAUNCH(k_b16_fill, grid_n((int64_t)N64 * N64), NT, 0, st)(M, N64);
+      EAR_LAUNCH(k_b16_clique, q->K, NT, 0, st)(LR, q->bcnt, q->boff, M, N64);
+      EAR_LAUNCH(k_b16_cross, grid_n(NB), NT, 0, st)(gv.rowptr, gv.col, gv.w, q->bvert, NB, q->reg, q->gidx, M, N64);
+      int per_sm = 0;
+      EAR_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_fw64, 256, 0));
+      const int T = N64 / F64;
+      const int gfw = (int)std::max<int64_t>(1, std::min<int64_t>((int64_t)T * (T + 1) / 2, (int64_t)per_sm * num_sms()));
+      int32_t NN = N64;
+      void *args[] = {(void *)&M, (void *)&NN};
+      count_launch();
+      EAR_CUDA_TRY(cudaLaunchCooperativeKernel((const void *)k_fw64, gfw, 256, args, 0, st));
+      int32_t *st2 = stats + 2;
+      EAR_LAUNCH(k_b16_narrow, grid_n((int64_t)NB * NBp), NT, 0, st)(M, N64, q->bvert, gv.cc, NB, NBp, dB16, st2, bad);
+      int32_t h_bad = 1;
+      EAR_TRY(rb1(&h_bad, bad, sizeof(int32_t), st, "part_solve"));
+      if (h_bad) EAR_CUDA_TRY(dev_memset(stats + 2, 0, sizeof(int32_t), st));   // the int32 FW redoes it
+      done = !h_bad;
+      tr.mark("dense boundary fw64");
     }
     if (!done) {   // dense: blocked FW over the boundary matrix
       int32_t *dB = nullptr, *labB = nullptr;

@@ -114,10 +114,11 @@ def test_reduced_D_equals_fw(pkg):
         assert torch.equal(D1, D2)
 
 
-@pytest.mark.parametrize("scale", [1, 100, 400])
+@pytest.mark.parametrize("scale", [1, 20, 40, 100, 400])
 def test_heavy_weights_fallback(pkg, scale):
-    """scale 100: distances up to ~0xFFFF -- the u16 sum bound fails and another route runs; scale 400:
-    distances beyond 0xFFFF.  Either way S is exact."""
+    """scale 20 / 40: boundary distances past the 64-tile FW's 0x7FFF cap (its int32 fallback) with the
+    products still in range; scale 100: distances up to ~0xFFFF -- the u16 sum bound fails and another
+    route runs; scale 400: distances beyond 0xFFFF.  Either way S is exact."""
     g0 = gg.torus(12, 12, 150, seed=3)
     g = Graph(g0.n, g0.src, g0.dst, (g0.w.astype(np.int64) * scale).astype(np.int32))
     out, ran = run(pkg, g, flags=pkg.FLAG_PART | pkg.FLAG_SSSP)
