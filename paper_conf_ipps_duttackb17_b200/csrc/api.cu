@@ -310,7 +310,9 @@ static ear_status_t solve_rows(ear_plan_s *p, int32_t row_begin, int32_t row_end
   const int32_t Np = padded(p, P);
   DKeep k;
   ear_status_t s = EAR_OK;
+  LabTrace tr(st, -3);
   if ((p->flags & EAR_FLAG_PART) && u16_ok && xp_applicable(p, st)) {
+    tr.mark("solve: xp lists");
     // Phase II by regions straight into u16 rows; every rank computes all of D (a few ms) and expands
     // only its own output rows, so no exchange is needed
     k.ld16 = xp_row_stride(p);
@@ -371,7 +373,9 @@ static ear_status_t solve_rows(ear_plan_s *p, int32_t row_begin, int32_t row_end
       if (s == EAR_OK) s = ear_gather_reduced(p, S, Np, k.D, Np, comm, st);
     }
   }
+  tr.mark("solve: phase II");
   if (s == EAR_OK && d_out) s = expand_kept(p, k, Np, row_begin, row_end, d_out, ldo, st);
+  tr.mark("solve: expansion");
   if (keep && s == EAR_OK) {
     *keep = k;
   } else {
@@ -393,7 +397,9 @@ ear_status_t apsp_full(int32_t n, int64_t m, const int32_t *d_src, const int32_t
     return EAR_EINVAL;
   }
   ear_plan_t p = nullptr;
+  LabTrace tr(st, -4);
   EAR_TRY(ear_decompose(n, m, d_src, d_dst, d_w, flags, stream, &p));
+  tr.mark("apsp_full: decompose");
   ear_status_t s = solve_rows(p, row_begin, row_end, d_out, ldo, comm, st, nullptr, rows_aligned(d_out, ldo));
   cudaError_t e = cudaStreamSynchronize(st);
   ear_plan_destroy(p);

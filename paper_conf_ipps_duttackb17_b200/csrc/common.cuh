@@ -1,7 +1,9 @@
 // Shared internals of libearapsp.so (product path only; nothing here is shared with oracle/).
 #pragma once
+#include <chrono>
 #include <cstdint>
 #include <cstdio>
+#include <cstdlib>
 #include <vector>
 #include <cuda_runtime.h>
 
@@ -109,6 +111,28 @@ struct ear_comm_s {
 };
 
 namespace ear {
+// EAR_PART_TRACE=1 (lab): host time at stage boundaries, each synchronised (stderr)
+struct LabTrace {
+  cudaStream_t st;
+  int depth;
+  bool on;
+  std::chrono::steady_clock::time_point t0;
+  LabTrace(cudaStream_t s, int d) : st(s), depth(d) {
+    static const bool env = getenv("EAR_PART_TRACE") != nullptr;
+    on = env;
+    if (on) {
+      cudaStreamSynchronize(st);
+      t0 = std::chrono::steady_clock::now();
+    }
+  }
+  void mark(const char *what) {
+    if (!on) return;
+    cudaStreamSynchronize(st);
+    const auto t = std::chrono::steady_clock::now();
+    fprintf(stderr, "[trace d%d] %-22s %8.3f ms\n", depth, what, std::chrono::duration<double, std::milli>(t - t0).count());
+    t0 = t;
+  }
+};
 // prof.cu
 enum ProfKind { PK_DECOMPOSE, PK_FW_INIT, PK_FW_P1, PK_FW_P2, PK_FW_P3, PK_COMM, PK_EXPAND, PK_SAME_CHAIN, PK_SSSP, PK_BCC, PK_COMPOSE,
                 PK_FW_P3_16, PK_FW16_CONV, PK_FW_SIDE_P1, PK_FW_SIDE_P2, PK_REREDUCE, PK_BCC_PREP, PK_EXPAND_D16,

@@ -1006,29 +1006,6 @@ __global__ void k_widen(const uint16_t *__restrict__ D16, int64_t ld16, int32_t 
   }
 }
 
-// EAR_PART_TRACE=1 (lab): host time at stage boundaries, each synchronised
-struct Trace {
-  cudaStream_t st;
-  int depth;
-  bool on;
-  std::chrono::steady_clock::time_point t0;
-  Trace(cudaStream_t s, int d) : st(s), depth(d) {
-    static const bool env = getenv("EAR_PART_TRACE") != nullptr;
-    on = env;
-    if (on) {
-      cudaStreamSynchronize(st);
-      t0 = std::chrono::steady_clock::now();
-    }
-  }
-  void mark(const char *what) {
-    if (!on) return;
-    cudaStreamSynchronize(st);
-    const auto t = std::chrono::steady_clock::now();
-    fprintf(stderr, "[part d%d] %-22s %8.3f ms\n", depth, what, std::chrono::duration<double, std::milli>(t - t0).count());
-    t0 = t;
-  }
-};
-
 struct Tmp {
   cudaStream_t st;
   std::vector<void *> ptrs;
@@ -1086,7 +1063,7 @@ ear_status_t part_build(const GView &gv, cudaStream_t st, ear_part_s **out) {
     return s;
   };
   const int g = grid_n(n);
-  Trace tr(st, -1);
+  LabTrace tr(st, -1);
   {
     int per_sm = 0;
     EAR_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_partition, NT, 0));
@@ -1154,9 +1131,12 @@ ear_status_t part_build(const GView &gv, cudaStream_t st, ear_part_s **out) {
 }
 
 static ear_status_t plan_view(ear_plan_s *p, cudaStream_t st, GView *gv) {
+  LabTrace tr(st, -2);
   EAR_TRY(sssp_prepare(p, st));
+  tr.mark("view: reduced CSR");
   const int32_t *cc = nullptr;
   EAR_TRY(reduced_labels(p, (int32_t)round_up(p->n_reduced, TILE), st, &cc));
+  tr.mark("view: components");
   *gv = GView{p->n_reduced, p->r_rowptr, p->r_col, p->r_w, cc};
   return EAR_OK;
 }
@@ -1185,7 +1165,7 @@ ear_status_t part_solve(const GView &gv, ear_part_s *q, uint16_t *out, int64_t l
   // mostly tiny components (K near n): the (column blocks x regions) product grid would dominate
   if (q->K > n / 16 && (double)q->K * ceil_div(n, MP_TC) > 65536.0) return EAR_OK;
   const int ps = depth == 0 ? prof_begin(PK_PART, st) : -1;
-  Trace tr(st, depth);
+  LabTrace tr(st, depth);
   Tmp t(st);
   uint16_t *LR = nullptr, *dB16 = nullptr, *DBVt = nullptr, *DBV = nullptr;
   int32_t *stats = nullptr;
