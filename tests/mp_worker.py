@@ -38,7 +38,7 @@ def main():
         r0, r1 = ea.row_block(g.n, world, rank)
         ref = oracle.apsp_rows(g.n, g.src, g.dst, g.w, np.arange(r0, r1))
         for flags in (0, ea.FLAG_FW32, ea.FLAG_BCC, ea.FLAG_SSSP, ea.FLAG_BCC | ea.FLAG_FW32,
-                      ea.FLAG_BCC | ea.FLAG_SSSP):
+                      ea.FLAG_BCC | ea.FLAG_SSSP, ea.FLAG_PART | ea.FLAG_BCC | ea.FLAG_SSSP):
             out = ea.apsp_full(g.n, dev(g.src), dev(g.dst), dev(g.w), row_begin=r0, row_end=r1, flags=flags,
                                comm=comm)
             torch.cuda.synchronize()

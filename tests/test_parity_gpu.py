@@ -194,11 +194,11 @@ def test_host_entry_point(pkg):
     assert_exact(out2.numpy(), oracle.apsp_rows(g.n, g.src, g.dst, g.w, np.arange(100, 1333)), "host rows")
 
 
-@pytest.mark.parametrize("flags", [0, "bcc"])
+@pytest.mark.parametrize("flags", [0, "bcc", "part"])
 def test_host_async_pipelined(pkg, flags):
     """apsp_full_host_async: two problems in flight at once (the second's Phases I-II overlap the
     first's row copies), into separate host buffers and, in order, into one shared buffer."""
-    fl = pkg.FLAG_BCC if flags == "bcc" else 0
+    fl = {"bcc": pkg.FLAG_BCC, "part": pkg.FLAG_PART, 0: 0}[flags]
     g1, g2 = gg.config("cfg1"), gg.corner_cases(77, n_target=900)
     r1, r2 = oracle.apsp(g1.n, g1.src, g1.dst, g1.w), oracle.apsp(g2.n, g2.src, g2.dst, g2.w)
     j1 = pkg.apsp_full_host_async(g1.n, g1.src, g1.dst, g1.w, flags=fl)
@@ -212,12 +212,13 @@ def test_host_async_pipelined(pkg, flags):
     assert_exact(shared.numpy(), r1, "async shared buffer")
 
 
-@pytest.mark.parametrize("flags", [0, "bcc"])
+@pytest.mark.parametrize("flags", [0, "bcc", "part"])
 def test_concurrent_host_threads(pkg, flags):
     """Two host threads, each on its own stream, solving different graphs at the same time: the
-    library's per-thread readback staging and its kernel memsets must not mix the two problems."""
+    library's per-thread readback staging and its kernel memsets must not mix the two problems (with
+    "part": two cooperative launches may be in flight at once)."""
     import threading
-    fl = pkg.FLAG_BCC if flags == "bcc" else 0
+    fl = {"bcc": pkg.FLAG_BCC, "part": pkg.FLAG_PART, 0: 0}[flags]
     gs = [gg.corner_cases(91, n_target=700), gg.torus(10, 14, 120, seed=4), gg.cycle(300, seed=5),
           gg.config("cfg1")]
     refs = [oracle.apsp(g.n, g.src, g.dst, g.w) for g in gs]
