@@ -58,7 +58,7 @@ enum {
                                hanging off it, joined through the articulation points; same D
                                bit for bit.  With EAR_FLAG_SSSP too, every big piece is reduced again
                                 and its reduced graph solved by the per-source SSSP instead of
-                               the FW (the bench's route: O(n m) work per piece instead of O(n^3)). */
+                               the FW (O(n m) work per piece instead of O(n^3)). */
   EAR_FLAG_PART = 16,       /* Phase II by regions (reading C24): G^r cut into connected
                                regions of <= 256 vertices (Voronoi cells of a multi-source BFS), the
                                distances inside every region by one CTA each, the distances between
@@ -137,6 +137,11 @@ void ear_plan_destroy(ear_plan_t plan);
  * aligned), Np = info.n_reduced_padded; padded vertices are isolated.
  * With EAR_FLAG_SSSP in the plan's flags, D is computed row by row by per-source label-correcting
  * SSSP on G^r instead (sharded: every rank its own rows, no communication until the gather).
+ * With EAR_FLAG_PART (single GPU, comm == NULL), D comes from the region route (regions,
+ * region FWs, the boundary graph, two min-plus products through the region boundaries
+ * generalised), computed as u16 rows and widened into d_D; when the route declines (distances too
+ * large for its u16 sums, or mostly tiny components) the route of the other flags runs.  apsp_full
+ * with EAR_FLAG_PART computes D by regions on every rank (no exchange) and expands the rank's rows.
  *   comm == NULL: d_D is the full Np x Np matrix.
  *   comm != NULL (P ranks, even P = 1): d_D holds this rank's OWNED TILE ROWS -- the 128-row blocks
  *                 ti with (ti mod 2P) in {rank, 2P-1-rank} (a zig-zag that balances the upper
