@@ -192,3 +192,38 @@ def test_expander_big_boundaries(pkg, n, deg):
     out, ran = run(pkg, g)
     exact(out.cpu().numpy(), oracle.apsp(g.n, g.src, g.dst, g.w), f"expander n={n}")
     assert ran
+
+
+def _g(n, edges, w=None):
+    s, d = (np.array(c, np.int32) for c in zip(*edges))
+    w = np.ones(len(s), np.int32) if w is None else np.asarray(w, np.int32)
+    return Graph(n, s, d, w)
+
+
+@pytest.mark.parametrize("case", ["star", "complete", "two_complete", "long_path", "unit_grid", "ladder"])
+def test_adversarial_shapes(pkg, case):
+    """shapes the Voronoi regions handle badly or trivially: a star (every leaf one hop from the hub: the
+    cell splitting runs down to one-vertex regions), complete graphs (every vertex a boundary vertex),
+    a 5,000-vertex path, a grid of unit weights (all ties), a ladder (two long parallel paths)"""
+    rng = np.random.default_rng(7)
+    if case == "star":
+        g = _g(701, [(0, i) for i in range(1, 701)], rng.integers(1, 50, 700))
+    elif case == "complete":
+        e = [(i, j) for i in range(300) for j in range(i + 1, 300)]
+        g = _g(300, e, rng.integers(1, 100, len(e)))
+    elif case == "two_complete":
+        e = [(i, j) for i in range(120) for j in range(i + 1, 120)]
+        e += [(120 + i, 120 + j) for i, j in e]
+        g = _g(240, e, rng.integers(1, 100, len(e)))
+    elif case == "long_path":
+        g = gg.path(5000, seed=3)
+    elif case == "unit_grid":
+        e = [(r * 40 + c, r * 40 + c + 1) for r in range(40) for c in range(39)]
+        e += [(r * 40 + c, (r + 1) * 40 + c) for r in range(39) for c in range(40)]
+        g = _g(1600, e)
+    else:
+        e = [(i, i + 1) for i in range(999)] + [(1000 + i, 1001 + i) for i in range(999)]
+        e += [(i, 1000 + i) for i in range(0, 1000, 7)]
+        g = _g(2000, e, rng.integers(1, 100, len(e)))
+    out, _ = run(pkg, g)
+    exact(out.cpu().numpy(), oracle.apsp(g.n, g.src, g.dst, g.w), case)
