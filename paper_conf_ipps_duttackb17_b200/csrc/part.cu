@@ -884,17 +884,22 @@ __global__ void __launch_bounds__(256) k_fw64(uint16_t *M, int32_t N) {
       __syncthreads();
     }
   };
-  for (int k = 0; k < T; ++k) {
-    if (blockIdx.x == 0) {
-      close_pivot(k);
+  auto store_tile = [&](int ti) {   // As -> tile (ti, ti)
 #pragma unroll
-      for (int q = 0; q < 4; ++q)
-        *reinterpret_cast<uint2 *>(M + (int64_t)(k * F64 + tr * 4 + q) * N + k * F64 + tc * 4) =
-            *reinterpret_cast<const uint2 *>(&As[tr * 4 + q][tc * 4]);
-    }
-    grid.sync();
-    if (blockIdx.x != 0 && blockIdx.x < T - 1) {
-      f64_load(As, M, N, k, k);   // the closed pivot tile
+    for (int q = 0; q < 4; ++q)
+      *reinterpret_cast<uint2 *>(M + (int64_t)(ti * F64 + tr * 4 + q) * N + ti * F64 + tc * 4) =
+          *reinterpret_cast<const uint2 *>(&As[tr * 4 + q][tc * 4]);
+  };
+  if (blockIdx.x == 0 && T > 0) {
+    close_pivot(0);
+    store_tile(0);
+  }
+  grid.sync();
+  for (int k = 0; k < T; ++k) {
+    // the closed pivot tile (stored before the last grid barrier by block 0)
+    if (blockIdx.x < T - 1) {
+      __syncthreads();
+      f64_load(As, M, N, k, k);
       __syncthreads();
     }
     // phase 2: pivot-row tiles (k, j) = min(C, P (x) C); P is closed and symmetric, so A[m][r] = P[m][r]
@@ -913,9 +918,44 @@ __global__ void __launch_bounds__(256) k_fw64(uint16_t *M, int32_t N) {
       f64_store(M, N, k, j, c, true);
     }
     grid.sync();
-    // phase 3: upper tiles (i <= j) off row / column k: C = min(C, row(k,i)^T (x) row(k,j)), mirrored
+    // phase 3: upper tiles (i <= j) off row / column k: C = min(C, row(k,i)^T (x) row(k,j)), mirrored.
+    // Lookahead: block 0 first updates the NEXT pivot tile (k+1, k+1) and closes it (phase 1 of round
+    // k+1) while the other blocks work through the rest of phase 3
+    if (blockIdx.x == 0 && k + 1 < T) {
+      __syncthreads();
+      f64_load(Bs, M, N, k, k + 1);
+      f64_load(As, M, N, k + 1, k + 1);
+      __syncthreads();
+      uint32_t c[4][2];
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        const uint2 x = *reinterpret_cast<const uint2 *>(&As[tr * 4 + q][tc * 4]);
+        c[q][0] = x.x, c[q][1] = x.y;
+      }
+      f64_mp(Bs, Bs, c);
+      __syncthreads();
+#pragma unroll
+      for (int q = 0; q < 4; ++q) *reinterpret_cast<uint2 *>(&As[tr * 4 + q][tc * 4]) = make_uint2(c[q][0], c[q][1]);
+      __syncthreads();
+      for (int kk = 0; kk < F64; ++kk) {   // close it in place (as close_pivot, from shared memory)
+        const uint2 bv = *reinterpret_cast<const uint2 *>(&As[kk][tc * 4]);
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+          const uint32_t a = dup16(As[tr * 4 + q][kk]);
+          uint2 cv = *reinterpret_cast<const uint2 *>(&As[tr * 4 + q][tc * 4]);
+          cv.x = __viaddmin_u16x2(a, bv.x, cv.x);
+          cv.y = __viaddmin_u16x2(a, bv.y, cv.y);
+          *reinterpret_cast<uint2 *>(&As[tr * 4 + q][tc * 4]) = cv;
+        }
+        __syncthreads();
+      }
+      store_tile(k + 1);
+    }
     const int64_t nt = (int64_t)T * (T + 1) / 2;
-    for (int64_t e = blockIdx.x; e < nt; e += gridDim.x) {
+    const int64_t skip = (int64_t)(k + 1) * (k + 2) / 2 + (k + 1);   // the tile (k+1, k+1): block 0 did it
+    const int gb = gridDim.x > 1 ? (int)gridDim.x - 1 : 1;            // block 0 takes regular tiles only alone
+    for (int64_t e = gridDim.x > 1 ? blockIdx.x - 1 : 0; e < nt && (gridDim.x == 1 || blockIdx.x > 0); e += gb) {
+      if (k + 1 < T && e == skip) continue;
       int i = (int)((sqrt(8.0 * (double)e + 1.0) - 1.0) / 2.0);   // e -> (j = row of the triangle, i <= j)
       while ((int64_t)(i + 1) * (i + 2) / 2 <= e) ++i;
       while ((int64_t)i * (i + 1) / 2 > e) --i;
