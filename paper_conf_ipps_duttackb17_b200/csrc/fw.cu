@@ -18,6 +18,7 @@
 // DESIGN.md sec. 6d).  Both run the same lookahead schedule: round k+1's pivot chain on a per-call side
 // stream while round k's remaining tiles proceed.  Every piece of per-call state (side stream, events,
 // tile counters, precheck word) belongs to the call, so distinct calls on one device are independent.
+#include <cooperative_groups.h>
 #include <cuda.h>
 #include <cudaTypedefs.h>
 #include <unistd.h>
@@ -820,26 +821,40 @@ __global__ void k_gather_pull(PeerPtrs regions, int32_t P, int32_t Np, int32_t *
 }
 
 // connected-component labels (min vertex id) of the reduced graph by hooking + pointer jumping
-__global__ void k_cc_init(int32_t *lab, int32_t n) {
-  for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x)
-    lab[v] = (int32_t)v;
-}
-__global__ void k_cc_hook(const int32_t *u, const int32_t *v, int64_t E, int32_t *lab, int32_t *changed) {
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < E; i += (int64_t)gridDim.x * blockDim.x) {
-    const int32_t a = lab[u[i]], b = lab[v[i]];
-    if (a != b) {
-      const int32_t hi = max(a, b), lo = min(a, b);
-      if (atomicMin(&lab[hi], lo) > lo) *changed = 1;
+// connected components of G^r in one cooperative launch: hooking of roots (smaller id wins) and pointer
+// jumping, separated by grid barriers, until a hooking pass changes nothing; labels = smallest vertex id
+// of the component.  st[0..2]: rotating per-pass change flags
+__global__ void k_cc_coop(const int32_t *__restrict__ u, const int32_t *__restrict__ v, int64_t E, int32_t *lab,
+                          int32_t n, int32_t *st) {
+  namespace cg = cooperative_groups;
+  cg::grid_group grid = cg::this_grid();
+  const int64_t tid0 = blockIdx.x * (int64_t)blockDim.x + threadIdx.x, stride = (int64_t)gridDim.x * blockDim.x;
+  for (int64_t x = tid0; x < n; x += stride) lab[x] = (int32_t)x;
+  if (tid0 == 0) st[0] = st[1] = st[2] = 0;
+  grid.sync();
+  for (int it = 0; it < 4 * 64; ++it) {
+    const int f = it % 3;
+    int ch = 0;
+    for (int64_t i = tid0; i < E; i += stride) {
+      const int32_t a = lab[u[i]], b = lab[v[i]];
+      if (a != b) {
+        const int32_t hi = max(a, b), lo = min(a, b);
+        if (atomicMin(&lab[hi], lo) > lo) ch = 1;
+      }
     }
+    if (__syncthreads_or(ch) && threadIdx.x == 0) st[f] = 1;
+    if (tid0 == 0) st[(it + 1) % 3] = 0;   // read two passes ago, before the last barrier
+    grid.sync();
+    for (int64_t x = tid0; x < n; x += stride) {
+      int32_t l = lab[x];
+      while (lab[l] != l) l = lab[l];
+      lab[x] = l;
+    }
+    grid.sync();
+    if (!st[f]) return;
   }
 }
-__global__ void k_cc_jump(int32_t *lab, int32_t n) {
-  for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
-    int32_t l = lab[v];
-    while (lab[l] != l) l = lab[l];
-    lab[v] = l;
-  }
-}
+
 
 // EAR_DEBUG_RACE_US (test knob, tests/test_concurrency_gpu.py): a device-side spin of that length ahead
 // of each cross-tile launch keeps the device behind the host, and a host sleep of the same length
@@ -1704,21 +1719,22 @@ ear_status_t reduced_labels(ear_plan_s *p, int32_t Np, cudaStream_t st, const in
     p->cc = nullptr;
     int32_t *changed = nullptr;
     EAR_CUDA_TRY(cudaMallocAsync((void **)&p->cc, sizeof(int32_t) * (size_t)Np, st));
-    EAR_CUDA_TRY(cudaMallocAsync((void **)&changed, sizeof(int32_t), st));
+    EAR_CUDA_TRY(cudaMallocAsync((void **)&changed, 4 * sizeof(int32_t), st));
     p->cc_np = Np;
-    EAR_LAUNCH(k_cc_init, grid_for(Np), 256, 0, st)(p->cc, Np);
     ear_status_t s = EAR_OK;
-    for (int it = 0; it < 64 && s == EAR_OK; ++it) {
-      int32_t h = 0;
-      if (p->n_redges == 0) break;
-      dev_memset(changed, 0, sizeof(int32_t), st);
-      EAR_LAUNCH(k_cc_hook, grid_for(p->n_redges), 256, 0, st)(p->re_u, p->re_v, p->n_redges, p->cc, changed);
-      EAR_LAUNCH(k_cc_jump, grid_for(Np), 256, 0, st)(p->cc, Np);
-      Readback rb(st);
-      cudaError_t e = rb.get(&h, changed, sizeof(int32_t));
-      if (e == cudaSuccess) e = rb.sync();
+    {
+      int per_sm = 0;
+      EAR_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_cc_coop, 256, 0));
+      const int64_t work = std::max<int64_t>(Np, p->n_redges);
+      const int g = (int)std::max<int64_t>(1, std::min<int64_t>(ceil_div(work, 256), (int64_t)per_sm * num_sms()));
+      const int32_t *ru = p->re_u, *rv = p->re_v;
+      int64_t E = p->n_redges;
+      int32_t *lab = p->cc, nn = Np;
+      void *args[] = {(void *)&ru, (void *)&rv, (void *)&E, (void *)&lab, (void *)&nn, (void *)&changed};
+      EAR_CUDA_TRY(dev_memset(changed, 0, 4 * sizeof(int32_t), st));
+      count_launch();
+      cudaError_t e = cudaLaunchCooperativeKernel((const void *)k_cc_coop, g, 256, args, 0, st);
       if (e != cudaSuccess) { set_error("reduced_labels: %s", cudaGetErrorString(e)); s = EAR_ECUDA; }
-      if (!h) break;
     }
     cudaFreeAsync(changed, st);
     EAR_TRY(s);
