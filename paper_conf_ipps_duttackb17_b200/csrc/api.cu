@@ -318,7 +318,7 @@ static ear_status_t solve_rows(ear_plan_s *p, int32_t row_begin, int32_t row_end
     k.ld16 = xp_row_stride(p);
     EAR_CUDA_TRY(cudaMallocAsync((void **)&k.D16, sizeof(uint16_t) * (size_t)p->n_reduced * k.ld16, st));
     bool applied = false;
-    s = part_rows(p, k.D16, k.ld16, nullptr, 0, 0, &applied, st);
+    s = part_rows(p, k.D16, k.ld16, nullptr, 0, 0, &applied, st, row_begin, row_end);
     if (s != EAR_OK || !applied) {
       cudaFreeAsync(k.D16, st);
       k.D16 = nullptr;

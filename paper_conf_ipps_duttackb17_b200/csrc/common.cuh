@@ -217,8 +217,10 @@ void bcc_free(ear_bcc_s *b, cudaStream_t stream);
 // part.cu -- Phase II by regions (EAR_FLAG_PART): every row of D as u16 into D16 (ld16 >= round_up(N_r, 8)),
 // or (D16 == NULL) widened into the int32 Np x Np matrix D; *applied = false when the route does not apply
 ear_status_t part_prepare(ear_plan_s *plan, cudaStream_t stream);
+// row_begin / row_end (D16 only): the caller's rows of G; D16 then holds only the rows Phase III stages
+// for them (the regions of their chain ends)
 ear_status_t part_rows(ear_plan_s *plan, uint16_t *D16, int64_t ld16, int32_t *D, int64_t ldd, int32_t Np,
-                       bool *applied, cudaStream_t stream);
+                       bool *applied, cudaStream_t stream, int32_t row_begin = 0, int32_t row_end = 0);
 void part_free(ear_part_s *q, cudaStream_t stream);
 // expand.cu
 ear_status_t expand(const ear_plan_s *plan, const int32_t *D, int64_t ldd, int32_t row_begin,

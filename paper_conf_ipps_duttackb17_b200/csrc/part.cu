@@ -324,9 +324,11 @@ __global__ void __launch_bounds__(MP_NT)
                 const int32_t *__restrict__ boff, const int32_t *__restrict__ perm, const uint16_t *__restrict__ Bsrc,
                 int64_t ldb, int32_t ncols, uint16_t *__restrict__ out, int64_t ldo, const int32_t *__restrict__ reg,
                 const int32_t *__restrict__ loc, const int32_t *__restrict__ cc, const int32_t *__restrict__ rcomp,
-                int32_t multi, const int32_t *__restrict__ rlist, const int32_t *__restrict__ stats) {
+                int32_t multi, const int32_t *__restrict__ rlist, const int32_t *__restrict__ stats,
+                const int32_t *__restrict__ rneed) {
   __shared__ __align__(16) uint32_t As[MP_KC][PCAP];
   if (stats[1] || stats[0] + stats[2] >= 0xFFFF || (FINAL && stats[0] + stats[3] >= 0xFFFF)) return;
+  if (rneed && !rneed[rlist ? rlist[blockIdx.y] : blockIdx.y]) return;
   __shared__ __align__(16) uint16_t Bs[MP_KC][MP_BS];
   __shared__ int32_t cl[MP_TC], ccol[MP_TC];
   const int i = rlist ? rlist[blockIdx.y] : blockIdx.y, tid = threadIdx.x;
@@ -610,14 +612,16 @@ constexpr int FINAL_SMEM = MP_KC * PCAP * 4 + 2 * MP_KC * FW_BS * 2;
 // item offsets of k_region_prod: region i contributes ceil(ncols / W_i) tiles (none when |B_i| > MP_KC:
 // the general kernel does it); one CTA, chunked block scan
 __global__ void __launch_bounds__(1024) k_items(const int32_t *__restrict__ roff, const int32_t *__restrict__ bcnt,
-                                                int32_t K, int32_t ncols, int32_t *itemoff) {
+                                                int32_t K, int32_t ncols, const int32_t *__restrict__ rneed,
+                                                int32_t *itemoff) {
   __shared__ int32_t part[1024];
   __shared__ int32_t carry;
   if (threadIdx.x == 0) carry = 0;
   for (int base = 0; base < K; base += 1024) {
     const int i = base + threadIdx.x;
     int32_t c = 0;
-    if (i < K && bcnt[i] <= MP_KC) c = (ncols + width_of(roff[i + 1] - roff[i]) - 1) / width_of(roff[i + 1] - roff[i]);
+    if (i < K && bcnt[i] <= MP_KC && (!rneed || rneed[i]))
+      c = (ncols + width_of(roff[i + 1] - roff[i]) - 1) / width_of(roff[i + 1] - roff[i]);
     part[threadIdx.x] = c;
     __syncthreads();
     for (int o = 1; o < 1024; o <<= 1) {   // inclusive Hillis-Steele scan
@@ -1029,6 +1033,21 @@ __global__ void k_b16_narrow(const uint16_t *__restrict__ M, int32_t N, const in
   if (__syncthreads_or(b) && threadIdx.x == 0) *bad = 1;
 }
 
+// rows a caller's output row range [rb, re) of G needs from D (Phase III stages them): the terminal's own
+// row, or both ends of a chain vertex; then the regions that hold one
+__global__ void k_need_rows(const VDesc *__restrict__ desc, int32_t rb, int32_t re, int32_t *need) {
+  for (int32_t s = rb + blockIdx.x * blockDim.x + threadIdx.x; s < re; s += gridDim.x * blockDim.x) {
+    const VDesc d = desc[s];
+    need[d.p] = 1;
+    need[d.q] = 1;
+  }
+}
+__global__ void k_need_regions(const int32_t *__restrict__ need, const int32_t *__restrict__ reg, int32_t n,
+                               int32_t *rneed) {
+  for (int32_t v = blockIdx.x * blockDim.x + threadIdx.x; v < n; v += gridDim.x * blockDim.x)
+    if (need[v]) rneed[reg[v]] = 1;
+}
+
 // int32 D (Np x Np, INF, padding isolated) from the u16 rows
 __global__ void k_widen(const uint16_t *__restrict__ D16, int64_t ld16, int32_t nr, int32_t *D, int64_t ldd,
                         int32_t Np) {
@@ -1199,7 +1218,7 @@ ear_status_t part_prepare(ear_plan_s *p, cudaStream_t st) {
 // *applied = false when the route does not apply (too many regions, a region distance or a sum that
 // could reach 0xFFFF); nothing is written then.  Profiled (PK_PART / PK_PART_MP) at depth 0 only.
 ear_status_t part_solve(const GView &gv, ear_part_s *q, uint16_t *out, int64_t ldo, int depth, bool fw32,
-                        bool *applied, cudaStream_t st) {
+                        bool *applied, cudaStream_t st, const int32_t *rneed = nullptr) {
   *applied = false;
   const int32_t n = gv.n;
   // mostly tiny components (K near n): the (column blocks x regions) product grid would dominate
@@ -1323,7 +1342,7 @@ ear_status_t part_solve(const GView &gv, ear_part_s *q, uint16_t *out, int64_t l
   EAR_CUDA_TRY(smem_attr((const void *)k_region_prod<false>, FINAL_SMEM));
   EAR_CUDA_TRY(smem_attr((const void *)k_region_prod<true>, FINAL_SMEM));
   if (NB > 0) {
-    EAR_LAUNCH(k_items, 1, 1024, 0, st)(q->roff, q->bcnt, q->K, NB, items);
+    EAR_LAUNCH(k_items, 1, 1024, 0, st)(q->roff, q->bcnt, q->K, NB, nullptr, items);
     EAR_LAUNCH(k_region_prod<false>, 2 * num_sms(), MP_NT, FINAL_SMEM, st)(LR, q->roff, q->bcnt, q->boff, q->perm, dB16,
                                                                           NBp, NB, DBVt, NBp, q->reg, q->loc, cc,
                                                                           q->rcomp, q->vrange, q->multi, items, q->K,
@@ -1331,7 +1350,8 @@ ear_status_t part_solve(const GView &gv, ear_part_s *q, uint16_t *out, int64_t l
     if (q->nbig > 0) {
       dim3 g1(NBp / MP_TC, q->nbig);
       EAR_LAUNCH(k_region_mp<false>, g1, MP_NT, 0, st)(LR, q->roff, q->bcnt, q->boff, q->perm, dB16, NBp, NBp, DBVt,
-                                                        NBp, q->reg, q->loc, cc, q->rcomp, q->multi, q->big, stats);
+                                                        NBp, q->reg, q->loc, cc, q->rcomp, q->multi, q->big, stats,
+                                                        nullptr);
     }
     if (!t.get(&DBV, (size_t)NB * ldv)) {
       set_error("part_solve: out of device memory");
@@ -1342,14 +1362,14 @@ ear_status_t part_solve(const GView &gv, ear_part_s *q, uint16_t *out, int64_t l
     EAR_LAUNCH(k_max16, grid_n((int64_t)NB * ldv / 8), NT, 0, st)(DBV, NB, ldv, n, stats + 3);
   }
   tr.mark("product1+T");
-  EAR_LAUNCH(k_items, 1, 1024, 0, st)(q->roff, q->bcnt, q->K, n, items);
+  EAR_LAUNCH(k_items, 1, 1024, 0, st)(q->roff, q->bcnt, q->K, n, rneed, items);
   EAR_LAUNCH(k_region_prod<true>, 2 * num_sms(), MP_NT, FINAL_SMEM, st)(LR, q->roff, q->bcnt, q->boff, q->perm, DBV,
                                                                        ldv, n, out, ldo, q->reg, q->loc, cc, q->rcomp,
                                                                        q->vrange, q->multi, items, q->K, stats);
   if (q->nbig > 0) {
     dim3 g2((unsigned)ceil_div(ldo, MP_TC), q->nbig);
     EAR_LAUNCH(k_region_mp<true>, g2, MP_NT, 0, st)(LR, q->roff, q->bcnt, q->boff, q->perm, DBVt, NBp, n, out, ldo,
-                                                     q->reg, q->loc, cc, q->rcomp, q->multi, q->big, stats);
+                                                     q->reg, q->loc, cc, q->rcomp, q->multi, q->big, stats, rneed);
   }
   if (pm >= 0) prof_end(pm, st, (double)n * q->sum_rb + (double)NB * q->sum_rb);
   int32_t h[4];
@@ -1363,7 +1383,7 @@ ear_status_t part_solve(const GView &gv, ear_part_s *q, uint16_t *out, int64_t l
 // Every row of D (reduced vertex order) as u16 (0xFFFF = INF, stride ld16 >= round_up(N_r, 8)), or
 // -- with D (int32, Np x Np, ldd) -- widened into it.  *applied = false when the route does not apply.
 ear_status_t part_rows(ear_plan_s *p, uint16_t *D16, int64_t ld16, int32_t *D, int64_t ldd, int32_t Np, bool *applied,
-                       cudaStream_t st) {
+                       cudaStream_t st, int32_t row_begin, int32_t row_end) {
   *applied = false;
   const int32_t n = p->n_reduced;
   if (n <= 0) return EAR_OK;
@@ -1380,7 +1400,19 @@ ear_status_t part_rows(ear_plan_s *p, uint16_t *D16, int64_t ld16, int32_t *D, i
       return EAR_ENOMEM;
     }
   }
-  EAR_TRY(part_solve(gv, p->part, out, ldo, 0, (p->flags & EAR_FLAG_FW32) != 0, applied, st));
+  int32_t *rneed = nullptr;   // a strict sub-range of G's rows: only the regions Phase III will stage
+  if (!D && (row_begin > 0 || row_end < p->n) && row_end > row_begin) {
+    int32_t *need = nullptr;
+    if (!t.get(&need, n) || !t.get(&rneed, p->part->K)) {
+      set_error("part_rows: out of device memory");
+      return EAR_ENOMEM;
+    }
+    EAR_CUDA_TRY(dev_memset(need, 0, sizeof(int32_t) * n, st));
+    EAR_CUDA_TRY(dev_memset(rneed, 0, sizeof(int32_t) * p->part->K, st));
+    EAR_LAUNCH(k_need_rows, grid_n(row_end - row_begin), NT, 0, st)(p->desc, row_begin, row_end, need);
+    EAR_LAUNCH(k_need_regions, grid_n(n), NT, 0, st)(need, p->part->reg, n, rneed);
+  }
+  EAR_TRY(part_solve(gv, p->part, out, ldo, 0, (p->flags & EAR_FLAG_FW32) != 0, applied, st, rneed));
   if (*applied && D) EAR_LAUNCH(k_widen, grid_n((int64_t)Np * Np), NT, 0, st)(out, ldo, n, D, ldd, Np);
   EAR_CUDA_TRY(cudaGetLastError());
   return EAR_OK;

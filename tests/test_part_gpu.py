@@ -227,3 +227,16 @@ def test_adversarial_shapes(pkg, case):
         g = _g(2000, e, rng.integers(1, 100, len(e)))
     out, _ = run(pkg, g)
     exact(out.cpu().numpy(), oracle.apsp(g.n, g.src, g.dst, g.w), case)
+
+
+@pytest.mark.parametrize("rng_rows", [(0, 1), (17, 18), (300, 700), (1499, 1500)])
+def test_row_ranges_need_only_their_regions(pkg, rng_rows):
+    """a strict row range computes only the regions Phase III stages for it (the chain ends of its rows):
+    several components, pendant paths and closed ears around the range edges"""
+    g = gg.corner_cases(5, n_target=1500)
+    a, b = rng_rows
+    b = min(b, g.n)
+    a = min(a, b - 1)
+    out, ran = run(pkg, g, rows=(a, b))
+    exact(out.cpu().numpy(), oracle.apsp_rows(g.n, g.src, g.dst, g.w, np.arange(a, b)), f"rows {a}:{b}")
+    assert ran
