@@ -79,6 +79,7 @@ constexpr int PSEED = 160;           // seed spacing (in vertex ids) of the firs
 constexpr uint32_t PC16 = 0x7FFF;    // cap of the region FW (two capped values never wrap)
 constexpr int FW_NT = 512;
 constexpr int MP_NT = 256, MP_TC = 128, MP_KC = 32, MP_BS = MP_TC + 8;   // Bs row stride (u16): 4-way max
+constexpr int PR_NT = 128, PR_MIN = 4;   // k_region_prod: 128 threads, 4 CTAs per SM (measured: 256 x 2 and 512 x 1 slower)
 constexpr int NT = 256;
 constexpr int PREC_MIN = 2048;      // a boundary graph this large is solved by regions again
 constexpr int PREC_DEPTH = 2;       // ... down to this nesting depth (then by the blocked FW)
@@ -455,11 +456,11 @@ __device__ __forceinline__ void cp_async_wait1() { asm volatile("cp.async.wait_g
 // for local columns.  Guard (uniform): nothing runs unless the u16 sums of this product cannot wrap,
 // stats[0] (Lmax) + stats[2] (max of dB) < 0xFFFF, for FINAL also stats[0] + stats[3] (max of DBV) <
 // 0xFFFF, and no region overflowed.
-constexpr int FW_MAXW = 512, FW_BS = FW_MAXW + 8;
-__device__ __forceinline__ int width_of(int32_t r) { return 16 * min(32, MP_NT / max(1, (r + 7) >> 3)); }
+constexpr int FW_MAXW = 128, FW_BS = FW_MAXW + 8;
+__device__ __forceinline__ int width_of(int32_t r) { return 16 * min(FW_MAXW / 16, PR_NT / max(1, (r + 7) >> 3)); }
 
 template <bool FINAL>
-__global__ void __launch_bounds__(MP_NT, 2)
+__global__ void __launch_bounds__(PR_NT, PR_MIN)
     k_region_prod(const uint16_t *__restrict__ LR, const int32_t *__restrict__ roff, const int32_t *__restrict__ bcnt,
                   const int32_t *__restrict__ boff, const int32_t *__restrict__ perm,
                   const uint16_t *__restrict__ Bsrc, int64_t ldb, int32_t ncols, uint16_t *__restrict__ out,
@@ -490,7 +491,7 @@ __global__ void __launch_bounds__(MP_NT, 2)
   auto issue = [&](int32_t t, int i, int32_t nb, int32_t b0, int32_t W, int buf) {
     const int32_t c0 = (t - itemoff[i]) * W;
     const int chunks = W / 8;
-    for (int e = tid; e < nb * chunks; e += MP_NT) {
+    for (int e = tid; e < nb * chunks; e += PR_NT) {
       const int k = e / chunks, c8 = (e % chunks) * 8;
       const bool ok = c0 + c8 < ldb;
       cp_async16(&Bs[buf][k][c8], Bsrc + (int64_t)(b0 + k) * ldb + (ok ? c0 + c8 : 0), ok ? 16 : 0);
@@ -516,18 +517,18 @@ __global__ void __launch_bounds__(MP_NT, 2)
       i_off = itemoff[i];
       if (FINAL) vr = vrange[i];
       const uint16_t *L = LR + (size_t)i * PCAP * PCAP;
-      for (int e = tid; e < nb * PCAP; e += MP_NT) {
+      for (int e = tid; e < nb * PCAP; e += PR_NT) {
         const int k = e / PCAP, u = e % PCAP;
         As[k][u] = u < r ? dup16(L[k * PCAP + u]) : 0xFFFFFFFFu;
       }
-      for (int u = tid; u < r; u += MP_NT) s_perm[u] = perm[r0 + u];
+      for (int u = tid; u < r; u += PR_NT) s_perm[u] = perm[r0 + u];
     }
     const int32_t c0 = (t - i_off) * W;
     int loc_any = 0;
     if (FINAL) {
       const bool meets = c0 <= vr.y && c0 + W > vr.x;
       if (meets || multi) {
-        for (int c = tid; c < W; c += MP_NT) {
+        for (int c = tid; c < W; c += PR_NT) {
           const int32_t v = c0 + c;
           int32_t lc = -1, cv = 0;
           if (v < ncols) {
@@ -1343,7 +1344,7 @@ ear_status_t part_solve(const GView &gv, ear_part_s *q, uint16_t *out, int64_t l
   EAR_CUDA_TRY(smem_attr((const void *)k_region_prod<true>, FINAL_SMEM));
   if (NB > 0) {
     EAR_LAUNCH(k_items, 1, 1024, 0, st)(q->roff, q->bcnt, q->K, NB, nullptr, items);
-    EAR_LAUNCH(k_region_prod<false>, 2 * num_sms(), MP_NT, FINAL_SMEM, st)(LR, q->roff, q->bcnt, q->boff, q->perm, dB16,
+    EAR_LAUNCH(k_region_prod<false>, (PR_MIN) * num_sms(), PR_NT, FINAL_SMEM, st)(LR, q->roff, q->bcnt, q->boff, q->perm, dB16,
                                                                           NBp, NB, DBVt, NBp, q->reg, q->loc, cc,
                                                                           q->rcomp, q->vrange, q->multi, items, q->K,
                                                                           stats);
@@ -1363,7 +1364,7 @@ ear_status_t part_solve(const GView &gv, ear_part_s *q, uint16_t *out, int64_t l
   }
   tr.mark("product1+T");
   EAR_LAUNCH(k_items, 1, 1024, 0, st)(q->roff, q->bcnt, q->K, n, rneed, items);
-  EAR_LAUNCH(k_region_prod<true>, 2 * num_sms(), MP_NT, FINAL_SMEM, st)(LR, q->roff, q->bcnt, q->boff, q->perm, DBV,
+  EAR_LAUNCH(k_region_prod<true>, (PR_MIN) * num_sms(), PR_NT, FINAL_SMEM, st)(LR, q->roff, q->bcnt, q->boff, q->perm, DBV,
                                                                        ldv, n, out, ldo, q->reg, q->loc, cc, q->rcomp,
                                                                        q->vrange, q->multi, items, q->K, stats);
   if (q->nbig > 0) {
