@@ -501,13 +501,14 @@ __global__ void __launch_bounds__(PR_NT, PR_MIN)
   __shared__ int32_t s_perm[PCAP];
   int cur = -1, buf = 0;
   int32_t r0 = 0, r = 0, nb = 0, b0 = 0, W = 16, cgs = 1, nro = 0, cgi = 0, ro = 0, i_off = 0;
+  int32_t i_end = itemoff[ri + 1];   // first item past region ri (kept in a register)
   int2 vr = make_int2(0, -1);
   {
     const int32_t rr = roff[ri + 1] - roff[ri];
     issue(t0, ri, bcnt[ri], boff[ri], width_of(rr), 0);
   }
   for (int32_t t = t0; t < t1; ++t) {
-    while (itemoff[ri + 1] <= t) ++ri;
+    while (i_end <= t) i_end = itemoff[++ri + 1];
     const int i = ri;
     __syncthreads();   // tile t-1 is done with As, Bs[buf ^ 1], cl, s_perm
     if (i != cur) {    // per-region constants and staging: A, the member ids
@@ -542,7 +543,7 @@ __global__ void __launch_bounds__(PR_NT, PR_MIN)
       }
     }
     if (t + 1 < t1) {
-      if (itemoff[i + 1] > t + 1) {
+      if (i_end > t + 1) {
         issue(t + 1, i, nb, b0, W, buf ^ 1);
       } else {
         int in = i + 1;
