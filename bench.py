@@ -403,10 +403,10 @@ def run_ours(args, rank, world, local_rank):
         ach = prof["part_minplus"] / (pm_ms / 1e3) / 1e12
         lanes = 2 * ALU_LANES_PER_SM
         peak_alu = SM_COUNT * lanes * sm_max * 1e6 / 1e12
-        roofline = {"bound": "alu", "kernel": "k_region_mp (Phase II by regions: min-plus products through the "
-                                              "region boundaries, packed u16x2)",
+        roofline = {"bound": "alu", "kernel": "k_region_prod (+ k_region_mp for boundaries > 32; Phase II by regions: "
+                                              "the two min-plus products through the region boundaries, packed u16x2)",
                     "achieved": ach, "peak": peak_alu, "unit": "Tminplus/s", "frac": ach / peak_alu,
-                    "traffic": ncu_traffic("k_region_mp", args.config), "avg_launch_ms": pm_ms / n_pm,
+                    "traffic": ncu_traffic("k_region_prod", args.config), "avg_launch_ms": pm_ms / n_pm,
                     "minplus_per_launch": prof["part_minplus"] / n_pm,
                     "peak_basis": f"{SM_COUNT} SMs x {lanes} min-plus/clk/SM (64 VIADDMNMX.U16x2, two lanes each) "
                                   f"x {sm_max:.0f} MHz (sm_max_mhz of MEASURED_PEAKS.json; issue rate from "
