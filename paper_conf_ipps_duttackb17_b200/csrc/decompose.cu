@@ -332,6 +332,7 @@ ear_status_t decompose(int32_t n, int64_t m, const int32_t *src, const int32_t *
   plan->flags = flags;
   plan->stream = st;
   Scratch S{st, {}};
+  LabTrace tr(st, -5);
 
   // ---- validation (reads the flags back at the N_r synchronisation point below; an invalid input
   //      must not be processed further, so we sync once here as well -- cheap).
@@ -355,6 +356,7 @@ ear_status_t decompose(int32_t n, int64_t m, const int32_t *src, const int32_t *
     return EAR_EOVERFLOW;
   }
 
+  tr.mark("decompose: validate");
   // ---- a1: arcs, sort, reduce-by-key(min)
   const int64_t M2 = 2 * m;
   const uint64_t sentinel = (uint64_t)(uint32_t)n << 32;
@@ -403,6 +405,7 @@ ear_status_t decompose(int32_t n, int64_t m, const int32_t *src, const int32_t *
     EAR_CUDA_TRY(cub::DeviceScan::ExclusiveSum(tmp, tb, deg, rowptr, n + 1, st));
   }
 
+  tr.mark("decompose: a1 sort/CSR");
   // ---- a2
   EAR_LAUNCH(k_terminals, grid_for(n), NT, 0, st)(deg, n, flags, term);
 
@@ -460,6 +463,7 @@ ear_status_t decompose(int32_t n, int64_t m, const int32_t *src, const int32_t *
   }
   plan->rank_rounds = total_rounds;
 
+  tr.mark("decompose: a2-a3 ranking");
   // ---- a4: terminal ids
   {
     size_t tb = 0;
@@ -555,6 +559,7 @@ ear_status_t decompose(int32_t n, int64_t m, const int32_t *src, const int32_t *
   EAR_CUDA_TRY(cudaGetLastError());
   EAR_CUDA_TRY(rbk.sync());
   if (plan->n_promoted < 0) plan->n_promoted = h_stats[0];
+  tr.mark("decompose: a4 + chains");
   return EAR_OK;
 }
 

@@ -1134,7 +1134,11 @@ ear_status_t part_build(const GView &gv, cudaStream_t st, ear_part_s **out) {
     void *args[] = {(void *)&rowptr, (void *)&col, (void *)&cc, (void *)&n, (void *)&S, (void *)&lab[0], (void *)&lab[1],
                     (void *)&grp, (void *)&cnt, (void *)&flags};
     count_launch();
-    EAR_CUDA_TRY(cudaLaunchCooperativeKernel((const void *)k_partition, gc, NT, args, 0, st));
+    if (cudaLaunchCooperativeKernel((const void *)k_partition, gc, NT, args, 0, st) != cudaSuccess) {
+      cudaGetLastError();
+      set_error("part_prepare: cooperative launch refused");
+      return fail(EAR_EUNSUPPORTED);   // the route does not apply (part_rows: another route runs)
+    }
   }
   const int cur = 0;
   tr.mark("build: bfs+split");
@@ -1202,6 +1206,7 @@ static ear_status_t plan_view(ear_plan_s *p, cudaStream_t st, GView *gv) {
   return EAR_OK;
 }
 
+// EAR_EUNSUPPORTED: no partition on this device (cooperative launches refused); callers fall back
 ear_status_t part_prepare(ear_plan_s *p, cudaStream_t st) {
   if (p->part) return EAR_OK;
   if (p->n_reduced <= 0) {
@@ -1279,10 +1284,13 @@ ear_status_t part_solve(const GView &gv, ear_part_s *q, uint16_t *out, int64_t l
       const GView hv{NB, hrow, hcol, hw, hcc};
       ear_part_s *qh = nullptr;
       tr.mark("H build");
-      EAR_TRY(part_build(hv, st, &qh));
-      ear_status_t s = part_solve(hv, qh, dB16, NBp, depth + 1, fw32, &done, st);
-      part_free(qh, st);
-      EAR_TRY(s);
+      const ear_status_t sb = part_build(hv, st, &qh);
+      if (sb != EAR_OK && sb != EAR_EUNSUPPORTED) return sb;
+      if (qh) {   // (no partition on this device: the dense FW below)
+        const ear_status_t s = part_solve(hv, qh, dB16, NBp, depth + 1, fw32, &done, st);
+        part_free(qh, st);
+        EAR_TRY(s);
+      }
       tr.mark("H solved");
       if (done) EAR_LAUNCH(k_max16, grid_n((int64_t)NB * NBp / 8), NT, 0, st)(dB16, NB, NBp, NB, stats + 2);
     }
@@ -1305,11 +1313,14 @@ ear_status_t part_solve(const GView &gv, ear_part_s *q, uint16_t *out, int64_t l
       int32_t NN = N64;
       void *args[] = {(void *)&M, (void *)&NN};
       count_launch();
-      EAR_CUDA_TRY(cudaLaunchCooperativeKernel((const void *)k_fw64, gfw, 256, args, 0, st));
-      int32_t *st2 = stats + 2;
-      EAR_LAUNCH(k_b16_narrow, grid_n((int64_t)NB * NBp), NT, 0, st)(M, N64, q->bvert, gv.cc, NB, NBp, dB16, st2, bad);
       int32_t h_bad = 1;
-      EAR_TRY(rb1(&h_bad, bad, sizeof(int32_t), st, "part_solve"));
+      if (cudaLaunchCooperativeKernel((const void *)k_fw64, gfw, 256, args, 0, st) == cudaSuccess) {
+        int32_t *st2 = stats + 2;
+        EAR_LAUNCH(k_b16_narrow, grid_n((int64_t)NB * NBp), NT, 0, st)(M, N64, q->bvert, gv.cc, NB, NBp, dB16, st2, bad);
+        EAR_TRY(rb1(&h_bad, bad, sizeof(int32_t), st, "part_solve"));
+      } else {
+        cudaGetLastError();   // no cooperative launch here (e.g. the device is shared): the blocked FW below
+      }
       if (h_bad) EAR_CUDA_TRY(dev_memset(stats + 2, 0, sizeof(int32_t), st));   // the int32 FW redoes it
       done = !h_bad;
       tr.mark("dense boundary fw64");
@@ -1389,7 +1400,11 @@ ear_status_t part_rows(ear_plan_s *p, uint16_t *D16, int64_t ld16, int32_t *D, i
   *applied = false;
   const int32_t n = p->n_reduced;
   if (n <= 0) return EAR_OK;
-  EAR_TRY(part_prepare(p, st));
+  {
+    const ear_status_t s = part_prepare(p, st);
+    if (s == EAR_EUNSUPPORTED) return EAR_OK;   // not applied: the caller's next route runs
+    EAR_TRY(s);
+  }
   GView gv;
   EAR_TRY(plan_view(p, st, &gv));
   Tmp t(st);
