@@ -541,7 +541,7 @@ def run_ours(args, rank, world, local_rank):
                 "ms_per_step": ms_max / K, "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
                 "dtype": ("int32 (SSSP: u16 shared-memory rows, exact below 0xFFFF; int32 fallback)"
                           if args.phase2 in ("sssp", "bcc_sssp") else
-                          "int32 (regions: packed u16x2 min-plus, exact while Dmax + 2 Lmax < 0xFFFF; other routes "
+                          "int32 (regions: packed u16x2 min-plus, exact while no u16 sum can reach 0x10000; other routes "
                           "otherwise)" if args.phase2 == "part" else
                           "int32" if prof["fw16_used"] == 0 else "int32 (FW: packed u16x2, exact below 0x7FFF)"),
                 "data": "synthetic (seeded generator, spatially coherent labels)",

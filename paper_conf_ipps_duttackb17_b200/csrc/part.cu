@@ -30,8 +30,9 @@
 // min-plus, against the per-source SSSP's N_r * M_r relaxations in hundreds of dependent rounds.
 //
 // Exactness: all distances are integers; the u16 lanes of VIADDMNMX.U16x2 add without saturation, so
-// the route is taken only when no sum of two operands of the same component can reach 0x10000:
-// Dmax + 2 Lmax < 0xFFFF (Lmax the largest d_i, Dmax the largest finite boundary distance).  Sums that
+// each product runs only when none of its sums of two operands of one component can reach 0x10000:
+// Lmax + max(dB) < 0xFFFF for (2), Lmax + max(DBV) < 0xFFFF for (1) (Lmax the largest d_i; the maxima
+// over finite entries, taken on the device and checked by the product kernels themselves).  Sums that
 // involve INF (0xFFFF, other components) wrap, but they only reach entries of pairs in different
 // components, which the last product overwrites with INF.  Otherwise *applied = false and the caller
 // runs another Phase II route.
