@@ -22,9 +22,13 @@
 //     boundary first; region / boundary offsets by scans;
 //   * k_region_fw: d_i for every region, one CTA per region, the PCAP x PCAP matrix in registers (8 x 16
 //     entries per thread as packed u16x2, one VIADDMNMX.U16x2 per two min-plus, capped at 0x7FFF);
-//   * the boundary matrix (cliques + joining arcs) and the blocked FW on it (fw_single, packed or int32);
-//   * k_region_mp<false>: (2) for every region j and every boundary column block -> DBVt[v][b] = d(b, v)
-//   * k_region_mp<true>: (1) for every region i and every 128-column block of D -> the u16 rows of D.
+//   * (3): the boundary graph H (cliques + joining arcs) solved by this same route when |B| >= PREC_MIN
+//     (nested), else densely by k_fw64 (one cooperative launch of a 64-tile FW, capped u16), with the
+//     blocked FW of fw.cu (int32) when a connected pair reaches the cap;
+//   * k_region_prod<false>: (2) for every region j and every boundary column tile -> DBVt[v][b] = d(b, v),
+//     then k_transpose16 -> DBV[b][v];
+//   * k_region_prod<true>: (1) for every region i and every column tile of D -> the u16 rows of D
+//     (k_region_mp: both products for regions whose boundary exceeds 32).
 // The two products are min-plus products with the region's boundary as the inner dimension
 // (K = |B_i|, ~10-40 on the paper's sparse graphs): dense work on the ALU pipe at N_r^2 * mean|B_i|
 // min-plus, against the per-source SSSP's N_r * M_r relaxations in hundreds of dependent rounds.
