@@ -98,6 +98,7 @@ extern "C" {
 
 ear_status_t ear_decompose(int32_t n, int64_t m, const int32_t *d_src, const int32_t *d_dst, const int32_t *d_w,
                            uint32_t flags, void *stream, ear_plan_t *out) {
+  NvtxRange nvtx_("ear: Phase I ear_decompose");
   g_err[0] = 0;
   keep_pool_memory();
   if (!out) { set_error("ear_decompose: out is NULL"); return EAR_EINVAL; }
@@ -164,6 +165,7 @@ void ear_plan_destroy(ear_plan_t p) {
 }
 
 ear_status_t apsp_reduced(ear_plan_t p, int32_t *d_D, int64_t ldd, ear_comm_t comm, void *stream) {
+  NvtxRange nvtx_("ear: Phase II apsp_reduced");
   g_err[0] = 0;
   if (!p || !d_D) { set_error("apsp_reduced: NULL argument"); return EAR_EINVAL; }
   const int32_t P = comm ? comm->nranks : 1;
@@ -260,6 +262,7 @@ ear_status_t ear_gather_reduced(ear_plan_t p, const int32_t *d_D_block, int64_t 
 
 ear_status_t expand_ears(ear_plan_t p, const int32_t *d_D_full, int64_t ldd, int32_t row_begin, int32_t row_end,
                          int32_t *d_out, int64_t ldo, void *stream) {
+  NvtxRange nvtx_("ear: Phase III expand_ears");
   g_err[0] = 0;
   if (!p || !d_D_full || (!d_out && row_end > row_begin)) { set_error("expand_ears: NULL argument"); return EAR_EINVAL; }
   if (row_begin < 0 || row_end < row_begin || row_end > p->n || ldo < p->n || ldd < p->n_reduced) {
@@ -272,6 +275,7 @@ ear_status_t expand_ears(ear_plan_t p, const int32_t *d_D_full, int64_t ldd, int
 
 ear_status_t ear_query_pairs(ear_plan_t p, const int32_t *d_D_full, int64_t ldd, int64_t npairs, const int32_t *d_s,
                              const int32_t *d_t, int32_t *d_out, void *stream) {
+  NvtxRange nvtx_("ear: query pairs");
   g_err[0] = 0;
   if (!p || !d_D_full || npairs < 0 || (npairs > 0 && (!d_s || !d_t || !d_out)) || ldd < p->n_reduced) {
     set_error("ear_query_pairs: bad argument");
@@ -306,6 +310,7 @@ static void free_kept(DKeep &k, cudaStream_t st) {
 // stores).  With `keep` D is handed back (not freed) for later expansions.
 static ear_status_t solve_rows(ear_plan_s *p, int32_t row_begin, int32_t row_end, int32_t *d_out, int64_t ldo,
                                ear_comm_t comm, cudaStream_t st, DKeep *keep, bool u16_ok) {
+  NvtxRange nvtx_("ear: Phases II + III");
   const int32_t P = comm ? comm->nranks : 1;
   const int32_t Np = padded(p, P);
   DKeep k;
@@ -391,6 +396,7 @@ static bool rows_aligned(const int32_t *out, int64_t ldo) {
 ear_status_t apsp_full(int32_t n, int64_t m, const int32_t *d_src, const int32_t *d_dst, const int32_t *d_w,
                        uint32_t flags, int32_t row_begin, int32_t row_end, int32_t *d_out, int64_t ldo,
                        ear_comm_t comm, void *stream) {
+  NvtxRange nvtx_("ear: apsp_full");
   cudaStream_t st = (cudaStream_t)stream;
   if (row_begin < 0 || row_end < row_begin || row_end > n || ldo < n) {
     set_error("apsp_full: bad row range [%d,%d) or ldo=%lld for n=%d", row_begin, row_end, (long long)ldo, n);
@@ -555,6 +561,7 @@ ear_status_t ear_job_wait(ear_job_t j) {
 ear_status_t apsp_full_host(int32_t n, int64_t m, const int32_t *h_src, const int32_t *h_dst, const int32_t *h_w,
                             uint32_t flags, int32_t row_begin, int32_t row_end, int32_t *h_out, int64_t ldo,
                             ear_comm_t comm, void *stream) {
+  NvtxRange nvtx_("ear: apsp_full_host");
   ear_job_t j = nullptr;
   EAR_TRY(apsp_full_host_async(n, m, h_src, h_dst, h_w, flags, row_begin, row_end, h_out, ldo, comm, stream, &j));
   ear_status_t s = ear_job_wait(j);

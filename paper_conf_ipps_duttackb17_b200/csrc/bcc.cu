@@ -864,6 +864,7 @@ static ear_status_t piece_rereduce(ear_plan_s *p, ear_bcc_s *b, int32_t id, int3
 ear_status_t bcc_solve(ear_plan_s *p, ear_comm_s *comm, int32_t *D, int64_t ldd, int32_t Np, int32_t row0,
                        int32_t rows, const int32_t *d_tile_rows, cudaStream_t st, uint16_t *D16, int64_t ld16,
                        int32_t *flag16) {
+  NvtxRange nvtx_("ear: Phase II by blocks");
   const int32_t P = comm ? comm->nranks : 1;
   int sb = prof_begin(PK_BCC_PREP, st);
   ear_status_t sprep = bcc_prepare(p, P, st);

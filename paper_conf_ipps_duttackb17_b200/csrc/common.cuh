@@ -6,6 +6,7 @@
 #include <cstdlib>
 #include <vector>
 #include <cuda_runtime.h>
+#include <nvtx3/nvToolsExt.h>
 
 #include "ear_apsp.h"
 
@@ -111,6 +112,14 @@ struct ear_comm_s {
 };
 
 namespace ear {
+// NVTX range around a phase of the path (visible in Nsight Systems / Compute timelines; header-only NVTX3,
+// a few ns when no tool is attached)
+struct NvtxRange {
+  explicit NvtxRange(const char *name) { nvtxRangePushA(name); }
+  ~NvtxRange() { nvtxRangePop(); }
+  NvtxRange(const NvtxRange &) = delete;
+  NvtxRange &operator=(const NvtxRange &) = delete;
+};
 // EAR_PART_TRACE=1 (lab): host time at stage boundaries, each synchronised (stderr)
 struct LabTrace {
   cudaStream_t st;

@@ -653,6 +653,7 @@ int32_t xp_gcap(int32_t nr) {
 // k_expand_pairs over u16 rows D16 (stride ld16) + the same-chain pass; the caller checked applicability
 ear_status_t launch_pairs(const ear_plan_s *plan, const uint16_t *D16, int32_t ld16, int32_t row_begin, int32_t row_end,
                           int32_t *out, int64_t ldo, cudaStream_t st, int prof_kind) {
+  NvtxRange nvtx_("ear: expansion (pair-major)");
   const ear_xp_s *x = plan->xp;
   const int32_t nr = plan->n_reduced, gcap = xp_gcap(nr);
   const int smem = (int)((1 + gcap) * (int64_t)ld16 * 2);

@@ -1579,6 +1579,7 @@ ear_status_t fw_init_D(const ear_plan_s *plan, int32_t *D, int64_t ldd, int32_t 
 // NULL) reached the cap; otherwise, or without allow16, the int32 schedule runs on D.
 ear_status_t fw_single(int32_t *D, int64_t ldd, int32_t Np, cudaStream_t st, const int32_t *lab, int32_t n_real,
                        bool allow16, ear_plan_s *plan) {
+  NvtxRange nvtx_("ear: blocked FW");
   FwCtx *ctx = nullptr;
   EAR_TRY(ctx_acquire(&ctx));
   CtxLease lease{ctx};

@@ -724,6 +724,7 @@ extern "C" {
 
 ear_status_t ear_mcb(int32_t n, int64_t m, const int32_t *d_src, const int32_t *d_dst, const int32_t *d_w, void *stream,
                      ear_mcb_t *out) {
+  NvtxRange nvtx_("ear: minimum cycle basis");
   if (!out) { set_error("ear_mcb: out is NULL"); return EAR_EINVAL; }
   *out = nullptr;
   if (n < 1 || m < 0 || (m > 0 && (!d_src || !d_dst || !d_w))) {

@@ -1110,6 +1110,7 @@ void part_free(ear_part_s *q, cudaStream_t st) {
 
 // The partition of a graph into regions (G^r: cached in the plan; the boundary graph: per solve).
 ear_status_t part_build(const GView &gv, cudaStream_t st, ear_part_s **out) {
+  NvtxRange nvtx_("ear: regions");
   *out = nullptr;
   const int32_t n = gv.n;
   const int32_t *rowptr = gv.rowptr, *col = gv.col, *cc = gv.cc;
@@ -1402,6 +1403,7 @@ ear_status_t part_solve(const GView &gv, ear_part_s *q, uint16_t *out, int64_t l
 // -- with D (int32, Np x Np, ldd) -- widened into it.  *applied = false when the route does not apply.
 ear_status_t part_rows(ear_plan_s *p, uint16_t *D16, int64_t ld16, int32_t *D, int64_t ldd, int32_t Np, bool *applied,
                        cudaStream_t st, int32_t row_begin, int32_t row_end) {
+  NvtxRange nvtx_("ear: Phase II by regions");
   *applied = false;
   const int32_t n = p->n_reduced;
   if (n <= 0) return EAR_OK;

@@ -1141,6 +1141,7 @@ static ear_status_t sssp16_rows(ear_plan_s *p, OutT *out, int64_t ldo, int32_t L
 }
 
 ear_status_t sssp_rows16(ear_plan_s *p, uint16_t *D16, int64_t ld16, bool *applied, cudaStream_t st) {
+  NvtxRange nvtx_("ear: Phase II by per-source SSSP");
   const int32_t L = (int32_t)round_up(std::max(p->n_reduced, 1), 8);
   if (ld16 < L) { *applied = false; return EAR_OK; }
   return sssp16_rows<uint16_t>(p, D16, ld16, L, 0, p->n_reduced, nullptr, applied, st);
