@@ -436,7 +436,7 @@ def run_ours(args, rank, world, local_rank):
 
     # Phase II alternatives (plain FW on all of G^r; SURVEY 8.f NEXT 2 per-source SSSP; NEXT 3 pieces)
     # (bit-identical D; reported beside the timed Phase II, not part of the timed steps)
-    alt = None
+    alt = fw_roof = None
     if world == 1 and not args.no_alt:
         alt = {"note": "Phase II only (D of G^r), one timed call after a warm-up call; --phase2 X times the full step"}
         for name, fl in (("fw", 0), ("sssp", ea.FLAG_SSSP), ("bcc", ea.FLAG_BCC), ("bcc_sssp", ea.FLAG_BCC | ea.FLAG_SSSP),
@@ -453,6 +453,24 @@ def run_ours(args, rank, world, local_rank):
             a1.record(stream)
             torch.cuda.synchronize()
             alt[f"{name}_phase2_ms"] = a0.elapsed_time(a1)
+            if name == "fw":   # the blocked FW of row a5: its phase-3 tile kernel against its ALU peak
+                ea.profile_reset()
+                ea.profile_enable(True)
+                ea.apsp_reduced(p2, D2)
+                torch.cuda.synchronize()
+                pf = ea.profile_read()
+                ea.profile_enable(False)
+                packed = pf["fw_phase3_16_minplus"] > 0
+                mp_ = pf["fw_phase3_16_minplus"] if packed else pf["fw_phase3_minplus"]
+                ms_ = pf["fw_phase3_16_ms"] if packed else pf["fw_phase3_ms"]
+                lanes_ = (2 if packed else 1) * ALU_LANES_PER_SM
+                pk = SM_COUNT * lanes_ * sm_max * 1e6 / 1e12
+                ach_ = mp_ / (ms_ / 1e3) / 1e12 if ms_ > 0 else 0.0
+                fw_roof = {"bound": "alu", "kernel": "k_fw_tiles<Frag16>" if packed else "k_fw_tiles<Frag32>",
+                           "route": "--phase2 fw (blocked FW on all of G^r, one apsp_reduced call)",
+                           "achieved": ach_, "peak": pk, "unit": "Tminplus/s", "frac": ach_ / pk if pk else None,
+                           "minplus": mp_, "phase3_ms": ms_,
+                           "traffic": ncu_traffic("k_fw_tiles<Frag16>" if packed else "k_fw_tiles<Frag32>", args.config)}
             del D2
             p2.destroy()
             torch.cuda.empty_cache()
@@ -554,7 +572,7 @@ def run_ours(args, rank, world, local_rank):
                            "phase2": args.phase2, "bcc": bcc, "part": part,
                            "l2": "inputs larger than L2 (D %.1f GB, output %.1f GB per step)" % (
                                4.0 * info.n_reduced_padded ** 2 / 1e9, 4.0 * g.n * g.n / 1e9)},
-                **rooflines,
+                **rooflines, "roofline_fw": fw_roof,
                 "fw_minplus_gops": fw_minplus / (fw_ms / 1e3) / 1e9 if fw_ms > 0 else None,
                 "phases_ms": phases, "phase2_alternatives": alt, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks,
                 "gpu_launches": launches, "step_ms": step_ms, "seeds": seeds,
