@@ -428,18 +428,25 @@ __global__ void __launch_bounds__(MP_NT)
 // DBV[g][v] = DBVt[v][g]: the boundary rows of d as the final product stages them (rows contiguous in v)
 constexpr int TR = 64;
 __global__ void k_transpose16(const uint16_t *__restrict__ in, int64_t ldi, int32_t rows, int32_t cols,
-                              uint16_t *__restrict__ out, int64_t ldo) {
+                              uint16_t *__restrict__ out, int64_t ldo, int32_t *mx_out) {
   __shared__ uint16_t tile[TR][TR + 2];
   const int r0 = blockIdx.y * TR, c0 = blockIdx.x * TR;
+  uint32_t mx = 0;   // largest entry < 0xFFFF (the no-wrap guard of product (1))
   for (int e = threadIdx.x; e < TR * TR; e += blockDim.x) {
     const int r = e / TR, c = e % TR;
-    if (r0 + r < rows && c0 + c < cols) tile[r][c] = in[(int64_t)(r0 + r) * ldi + c0 + c];
+    if (r0 + r < rows && c0 + c < cols) {
+      const uint16_t x = in[(int64_t)(r0 + r) * ldi + c0 + c];
+      tile[r][c] = x;
+      if (x != 0xFFFF) mx = max(mx, (uint32_t)x);
+    }
   }
   __syncthreads();
   for (int e = threadIdx.x; e < TR * TR; e += blockDim.x) {
     const int c = e / TR, r = e % TR;
     if (r0 + r < rows && c0 + c < cols) out[(int64_t)(c0 + c) * ldo + r0 + r] = tile[r][c];
   }
+  for (int o = 16; o; o >>= 1) mx = max(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+  if ((threadIdx.x & 31) == 0 && mx) atomicMax(mx_out, (int32_t)mx);
 }
 
 __device__ __forceinline__ void cp_async16(void *smem, const void *gmem, int bytes) {
@@ -1377,8 +1384,7 @@ ear_status_t part_solve(const GView &gv, ear_part_s *q, uint16_t *out, int64_t l
       return EAR_ENOMEM;
     }
     dim3 gt((unsigned)ceil_div(NB, TR), (unsigned)ceil_div(n, TR));
-    EAR_LAUNCH(k_transpose16, gt, NT, 0, st)(DBVt, NBp, n, NB, DBV, ldv);
-    EAR_LAUNCH(k_max16, grid_n((int64_t)NB * ldv / 8), NT, 0, st)(DBV, NB, ldv, n, stats + 3);
+    EAR_LAUNCH(k_transpose16, gt, NT, 0, st)(DBVt, NBp, n, NB, DBV, ldv, stats + 3);
   }
   tr.mark("product1+T");
   EAR_LAUNCH(k_items, 1, 1024, 0, st)(q->roff, q->bcnt, q->K, n, rneed, items);
