@@ -133,3 +133,34 @@ def test_cfg5_full_matrix_certified(route):
     torch.cuda.empty_cache()
     report(s)
     assert s["violations"] == 0, s
+
+
+@pytest.mark.skipif(os.environ.get("EAR_VERIFY_CFG5") != "1", reason="cfg5 full check: EAR_VERIFY_CFG5=1 (~3 min)")
+def test_cfg5_one_call_one_gpu_certified():
+    """The north-star size in ONE apsp_full call on ONE B200: cfg5's whole 200k x 200k int32 matrix (160 GB)
+    resident in HBM beside the region route's working set, timed, then every entry certified."""
+    import paper_conf_ipps_duttackb17_b200 as ea
+    g = gg.config("cfg5")
+    free, total = torch.cuda.mem_get_info()
+    need = 4 * g.n * g.n
+    if free < need + 12 * 2**30:
+        pytest.skip(f"{free / 2**30:.0f} GiB free of {total / 2**30:.0f}: the 149 GiB output does not fit beside the rest")
+    src, dst, w = dev(g.src), dev(g.dst), dev(g.w)
+    out = torch.empty((g.n, g.n), dtype=torch.int32, device="cuda")
+    fl = ea.FLAG_PART | ea.FLAG_BCC | ea.FLAG_SSSP
+    ea.apsp_full(g.n, src, dst, w, out=out, flags=fl)   # warm-up (module load, pools)
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record()
+    ea.apsp_full(g.n, src, dst, w, out=out, flags=fl)
+    e1.record()
+    torch.cuda.synchronize()
+    ms = e0.elapsed_time(e1)
+    s = certify_stream(g, lambda r0, r1: out[r0:r1], 10000)
+    s.update({"config": "cfg5", "n": g.n, "m": g.m, "path": "apsp_full FLAG_PART, ONE call, 160 GB output on one B200",
+              "gpu_apsp_full_ms": ms, "entries_per_s": g.n * g.n / (ms / 1e3),
+              "hbm_free_gib_before": free / 2**30, "hbm_total_gib": total / 2**30})
+    del out
+    torch.cuda.empty_cache()
+    report(s)
+    assert s["violations"] == 0, s
