@@ -335,6 +335,7 @@ __global__ void k_xp_pairs(int32_t nc, const uint64_t *key, const int32_t *head,
     }
 }
 __global__ void k_xp_last(int32_t np, int32_t nc, int32_t *pstart) { pstart[np] = nc; }
+__global__ void k_xp_last_dev(const int32_t *np, int32_t nc, int32_t *pstart) { pstart[*np] = nc; }
 __global__ void k_xp_tid2v(int32_t n, const int32_t *tid, int32_t *tid2v) {
   for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x)
     if (tid[v] >= 0) tid2v[tid[v]] = (int32_t)v;
@@ -548,7 +549,7 @@ __global__ void __launch_bounds__(XP_NT, 1)
 
 struct ear_xp_s {
   int32_t ok = 0;            // the pair-major layout applies to this plan
-  int32_t npairs = 0, nc = 0;
+  int32_t npairs = 0, nc = 0;   // npairs: not read back (pstart / px are sized by nc)
   uint2 *pd = nullptr;       // [n] packed descriptors {p | q << 16, cp | cq << 16}
   int32_t *rows = nullptr;   // [nc] chain vertices sorted by (smaller end, larger end, chain, offset)
   int32_t *pstart = nullptr; // [npairs + 1]
@@ -617,13 +618,11 @@ ear_status_t xp_build(ear_plan_s *p, cudaStream_t st) {
     if (dv.Current() != x->rows) EAR_CUDA_TRY(dev_copy(x->rows, dv.Current(), sizeof(int32_t) * nc, st));
     EAR_LAUNCH(k_xp_heads, g(nc), 256, 0, st)(nc, dk.Current(), head);
     EAR_CUDA_TRY(cub::DeviceScan::InclusiveSum(tmp, tb2, head, hscan, nc, st));
-    Readback rb(st);
-    EAR_CUDA_TRY(rb.get(&npairs, hscan + nc - 1, sizeof(int32_t)));
-    EAR_CUDA_TRY(rb.sync());
-    EAR_CUDA_TRY(cudaMallocAsync((void **)&x->pstart, sizeof(int32_t) * ((size_t)npairs + 1), st));
-    EAR_CUDA_TRY(cudaMallocAsync((void **)&x->px, sizeof(int32_t) * (size_t)std::max(npairs, 1), st));
+    // pairs <= chain vertices: sized by nc, so no host round trip for the pair count
+    EAR_CUDA_TRY(cudaMallocAsync((void **)&x->pstart, sizeof(int32_t) * ((size_t)nc + 1), st));
+    EAR_CUDA_TRY(cudaMallocAsync((void **)&x->px, sizeof(int32_t) * (size_t)std::max(nc, 1), st));
     EAR_LAUNCH(k_xp_pairs, g(nc), 256, 0, st)(nc, dk.Current(), head, hscan, x->pstart, x->px, pcount);
-    EAR_LAUNCH(k_xp_last, 1, 1, 0, st)(npairs, nc, x->pstart);
+    EAR_LAUNCH(k_xp_last_dev, 1, 1, 0, st)(hscan + nc - 1, nc, x->pstart);
     EAR_CUDA_TRY(cub::DeviceScan::ExclusiveSum(tmp, tb3, pcount, x->istart, nr + 1, st));
   } else {
     EAR_CUDA_TRY(cudaMallocAsync((void **)&x->pstart, sizeof(int32_t), st));
