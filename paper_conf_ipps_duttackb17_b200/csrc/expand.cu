@@ -384,7 +384,10 @@ __device__ __forceinline__ int32_t out_v(int32_t cp, int32_t rp, int32_t cq, int
   return CONN ? __viaddmin_s32(cq, rq, cp + rp) : out_val(cp, rp, cq, rq);
 }
 
-template <bool CONN>
+// GP (global partners): rows too long for two in shared memory (cfg5: 120 KB per u16 row): only the
+// item's row is staged; the partners' rows are gathered from D16 in global memory (L2-resident while
+// the sweep runs), up to gcap = XP_GMAX of them per sweep
+template <bool CONN, bool GP>
 __global__ void __launch_bounds__(XP_NT, 1)
     k_expand_pairs(const uint16_t *__restrict__ D16, int32_t ldr, int32_t nr, const VDesc *__restrict__ desc,
                    const XpView X, int32_t n, int32_t rb, int32_t re, int32_t *__restrict__ out, int64_t ldo,
@@ -474,10 +477,11 @@ __global__ void __launch_bounds__(XP_NT, 1)
         if (!loaded_v)
           for (int i = tid; i < nv; i += XP_NT)
             reinterpret_cast<uint4 *>(srow)[i] = reinterpret_cast<const uint4 *>(D16 + (int64_t)v * ldr)[i];
-        for (int k = 0; k < ns; ++k)
-          for (int i = tid; i < nv; i += XP_NT)
-            reinterpret_cast<uint4 *>(srow + (1 + k) * ldr)[i] =
-                reinterpret_cast<const uint4 *>(D16 + (int64_t)slot_x[k] * ldr)[i];
+        if (!GP)
+          for (int k = 0; k < ns; ++k)
+            for (int i = tid; i < nv; i += XP_NT)
+              reinterpret_cast<uint4 *>(srow + (1 + k) * ldr)[i] =
+                  reinterpret_cast<const uint4 *>(D16 + (int64_t)slot_x[k] * ldr)[i];
         loaded_v = true;
         __syncthreads();
         // descriptors of the next column group are loaded while the current one is computed and stored
@@ -517,7 +521,7 @@ __global__ void __launch_bounds__(XP_NT, 1)
 #pragma unroll
               for (int j = 0; j < 4; ++j) Rx[j] = Rv[j];
             } else {
-              r_of<CONN>(srow + R.x * ldr, pq, cc, Rx);
+              r_of<CONN>(GP ? D16 + (int64_t)slot_x[R.x - 1] * ldr : srow + R.x * ldr, pq, cc, Rx);
             }
             for (int r = R.y; r < R.z; ++r) {
               const int4 m = meta[r];
@@ -638,6 +642,16 @@ ear_status_t xp_build(ear_plan_s *p, cudaStream_t st) {
   return EAR_OK;
 }
 
+// the item's own u16 row of D fits in a CTA's shared memory
+bool xp_row_fits(int32_t nr) {
+  int dev = 0, smax = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess || cudaDeviceGetAttribute(&smax, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev) != cudaSuccess) {
+    cudaGetLastError();
+    return false;
+  }
+  return round_up(std::max(nr, 1), 8) * 2 <= (int64_t)smax - 4096;
+}
+
 // partner rows that fit in shared memory beside the item's own row (0: the pair-major layout does not fit)
 int32_t xp_gcap(int32_t nr) {
   int dev = 0, smax = 0;
@@ -654,22 +668,34 @@ ear_status_t launch_pairs(const ear_plan_s *plan, const uint16_t *D16, int32_t l
                           int32_t *out, int64_t ldo, cudaStream_t st, int prof_kind) {
   NvtxRange nvtx_("ear: expansion (pair-major)");
   const ear_xp_s *x = plan->xp;
-  const int32_t nr = plan->n_reduced, gcap = xp_gcap(nr);
-  const int smem = (int)((1 + gcap) * (int64_t)ld16 * 2);
+  const int32_t nr = plan->n_reduced;
+  // one row per CTA, partners gathered from global memory (EAR_XP_GP=1: always, for tests)
+  const char *force = getenv("EAR_XP_GP");
+  const bool gp = xp_gcap(nr) < 1 || (force && atoi(force) == 1);
+  const int32_t gcap = gp ? XP_GMAX : xp_gcap(nr);
+  const int smem = (int)((gp ? 1 : 1 + gcap) * (int64_t)ld16 * 2);
   const bool conn = plan->connected == 1;
-  EAR_CUDA_TRY(smem_attr(conn ? (const void *)k_expand_pairs<true> : (const void *)k_expand_pairs<false>, smem));
+  const void *kf = gp ? (conn ? (const void *)k_expand_pairs<true, true> : (const void *)k_expand_pairs<false, true>)
+                      : (conn ? (const void *)k_expand_pairs<true, false> : (const void *)k_expand_pairs<false, false>);
+  EAR_CUDA_TRY(smem_attr(kf, smem));
   int32_t *counter = nullptr;
   EAR_CUDA_TRY(cudaMallocAsync((void **)&counter, sizeof(int32_t), st));
   EAR_CUDA_TRY(dev_memset(counter, 0, sizeof(int32_t), st));
   const XpView V{x->pd, x->rows, x->pstart, x->px, x->istart, x->tid2v};
   const double rows = row_end - row_begin;
   int se = prof_begin(prof_kind, st);
-  if (conn)
-    EAR_LAUNCH(k_expand_pairs<true>, num_sms(), XP_NT, smem, st)(D16, ld16, nr, plan->desc, V, plan->n, row_begin,
-                                                                  row_end, out, ldo, gcap, counter);
+  if (gp && conn)
+    EAR_LAUNCH((k_expand_pairs<true, true>), num_sms(), XP_NT, smem, st)(D16, ld16, nr, plan->desc, V, plan->n,
+                                                                          row_begin, row_end, out, ldo, gcap, counter);
+  else if (gp)
+    EAR_LAUNCH((k_expand_pairs<false, true>), num_sms(), XP_NT, smem, st)(D16, ld16, nr, plan->desc, V, plan->n,
+                                                                           row_begin, row_end, out, ldo, gcap, counter);
+  else if (conn)
+    EAR_LAUNCH((k_expand_pairs<true, false>), num_sms(), XP_NT, smem, st)(D16, ld16, nr, plan->desc, V, plan->n,
+                                                                           row_begin, row_end, out, ldo, gcap, counter);
   else
-    EAR_LAUNCH(k_expand_pairs<false>, num_sms(), XP_NT, smem, st)(D16, ld16, nr, plan->desc, V, plan->n, row_begin,
-                                                                   row_end, out, ldo, gcap, counter);
+    EAR_LAUNCH((k_expand_pairs<false, false>), num_sms(), XP_NT, smem, st)(D16, ld16, nr, plan->desc, V, plan->n,
+                                                                            row_begin, row_end, out, ldo, gcap, counter);
   // algorithmic bytes: the output, D read once (counted as the int32 D, as for the row-group kernel), the
   // descriptors
   prof_end(se, st, 4.0 * rows * plan->n + 16.0 * plan->n + 4.0 * (double)nr * nr * rows / plan->n);
@@ -731,7 +757,8 @@ int32_t xp_row_stride(const ear_plan_s *plan) { return (int32_t)round_up(std::ma
 bool xp_applicable(ear_plan_s *plan, cudaStream_t st) {
   const char *env = getenv("EAR_EXPAND_PAIRS");   // 0: the row-group kernel (A/B)
   if (env && atoi(env) == 0) return false;
-  if (plan->n_reduced >= 0xFFFF || xp_gcap(plan->n_reduced) < 1) return false;
+  // one row beside the item's (gcap >= 1), or -- partners then gathered from global memory -- the item's row alone
+  if (plan->n_reduced >= 0xFFFF || !xp_row_fits(plan->n_reduced)) return false;
   if (!plan->xp && xp_build(plan, st) != EAR_OK) {
     cudaGetLastError();
     return false;

@@ -240,3 +240,15 @@ def test_row_ranges_need_only_their_regions(pkg, rng_rows):
     out, ran = run(pkg, g, rows=(a, b))
     exact(out.cpu().numpy(), oracle.apsp_rows(g.n, g.src, g.dst, g.w, np.arange(a, b)), f"rows {a}:{b}")
     assert ran
+
+
+@pytest.mark.parametrize("case", ["cfg2", "corner", "cfg2_random"])
+def test_expansion_global_partners(pkg, case, monkeypatch):
+    """the pair-major expansion with only the item's row in shared memory and the partners' rows gathered
+    from global memory (cfg5's 120 KB rows need it), forced on small graphs by EAR_XP_GP=1"""
+    monkeypatch.setenv("EAR_XP_GP", "1")
+    g = {"cfg2": lambda: gg.config("cfg2"), "corner": lambda: gg.corner_cases(17, n_target=1800),
+         "cfg2_random": lambda: gg.config("cfg2", labels="random")}[case]()
+    for flags in (pkg.FLAG_PART, pkg.FLAG_BCC):
+        out, _ = run(pkg, g, flags=flags)
+        exact(out.cpu().numpy(), oracle.apsp(g.n, g.src, g.dst, g.w), f"{case} flags={flags}")
