@@ -384,11 +384,13 @@ __device__ __forceinline__ int32_t out_v(int32_t cp, int32_t rp, int32_t cq, int
   return CONN ? __viaddmin_s32(cq, rq, cp + rp) : out_val(cp, rp, cq, rq);
 }
 
-// GP (global partners): rows too long for two in shared memory (cfg5: 120 KB per u16 row): only the
-// item's row is staged; the partners' rows are gathered from D16 in global memory (L2-resident while
-// the sweep runs), up to gcap = XP_GMAX of them per sweep
-template <bool CONN, bool GP>
-__global__ void __launch_bounds__(XP_NT, 1)
+// GP (global partners): only the item's row is staged; the partners' rows are gathered from D16 in
+// global memory (L2-resident while the sweep runs), up to gcap = XP_GMAX of them per sweep.  With one row
+// per CTA two 512-thread CTAs share an SM (cfg4: 60 KB rows), so one's sweep building and row staging
+// overlap the other's column loop (measured 8.87 -> 8.47 ms on cfg4); rows too long for two per SM
+// (cfg5: 120 KB) run one 1024-thread CTA per SM.  !GP: the partners' rows staged beside the item's.
+template <bool CONN, bool GP, int NTT>
+__global__ void __launch_bounds__(NTT, 1024 / NTT)
     k_expand_pairs(const uint16_t *__restrict__ D16, int32_t ldr, int32_t nr, const VDesc *__restrict__ desc,
                    const XpView X, int32_t n, int32_t rb, int32_t re, int32_t *__restrict__ out, int64_t ldo,
                    int32_t gcap, int32_t *counter) {
@@ -475,11 +477,11 @@ __global__ void __launch_bounds__(XP_NT, 1)
       if (nrow > 0 || need_term) {
         const int nv = (nr + 7) / 8;   // 16-byte vectors per row
         if (!loaded_v)
-          for (int i = tid; i < nv; i += XP_NT)
+          for (int i = tid; i < nv; i += NTT)
             reinterpret_cast<uint4 *>(srow)[i] = reinterpret_cast<const uint4 *>(D16 + (int64_t)v * ldr)[i];
         if (!GP)
           for (int k = 0; k < ns; ++k)
-            for (int i = tid; i < nv; i += XP_NT)
+            for (int i = tid; i < nv; i += NTT)
               reinterpret_cast<uint4 *>(srow + (1 + k) * ldr)[i] =
                   reinterpret_cast<const uint4 *>(D16 + (int64_t)slot_x[k] * ldr)[i];
         loaded_v = true;
@@ -490,7 +492,7 @@ __global__ void __launch_bounds__(XP_NT, 1)
           na = *reinterpret_cast<const uint4 *>(X.pd + tid * 4);
           nb4 = *reinterpret_cast<const uint4 *>(X.pd + tid * 4 + 2);
         }
-        for (int32_t c0 = tid * 4; c0 < n; c0 += XP_NT * 4) {
+        for (int32_t c0 = tid * 4; c0 < n; c0 += NTT * 4) {
           uint32_t pq[4], cc[4];
           const bool full = c0 + 4 <= n;
           if (full) {
@@ -502,7 +504,7 @@ __global__ void __launch_bounds__(XP_NT, 1)
               pq[j] = q.x; cc[j] = q.y;
             }
           }
-          const int32_t c1 = c0 + XP_NT * 4;
+          const int32_t c1 = c0 + NTT * 4;
           if (c1 + 4 <= n) {
             na = *reinterpret_cast<const uint4 *>(X.pd + c1);
             nb4 = *reinterpret_cast<const uint4 *>(X.pd + c1 + 2);
@@ -669,14 +671,23 @@ ear_status_t launch_pairs(const ear_plan_s *plan, const uint16_t *D16, int32_t l
   NvtxRange nvtx_("ear: expansion (pair-major)");
   const ear_xp_s *x = plan->xp;
   const int32_t nr = plan->n_reduced;
-  // one row per CTA, partners gathered from global memory (EAR_XP_GP=1: always, for tests)
-  const char *force = getenv("EAR_XP_GP");
-  const bool gp = xp_gcap(nr) < 1 || (force && atoi(force) == 1);
+  // GP with two 512-thread CTAs per SM when two single-row CTAs fit an SM's shared memory, GP with one
+  // 1024-thread CTA when only one row fits beside nothing else, the partners staged otherwise (never: a
+  // row that fits twice in a CTA fits twice in an SM).
+  int dev = 0, per_sm = 0;
+  EAR_CUDA_TRY(cudaGetDevice(&dev));
+  EAR_CUDA_TRY(cudaDeviceGetAttribute(&per_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, dev));
+  const int64_t rowb = (int64_t)ld16 * 2;
+  const char *force = getenv("EAR_XP_GP");   // tests: 0 staged partners, 1 global (two CTAs/SM), 2 global (one)
+  const int fv = force ? atoi(force) : -1;
+  const bool two = 2 * (rowb + 4096) <= per_sm && fv != 2;
+  const bool gp = fv >= 0 ? fv >= 1 : (two || xp_gcap(nr) < 1);
   const int32_t gcap = gp ? XP_GMAX : xp_gcap(nr);
-  const int smem = (int)((gp ? 1 : 1 + gcap) * (int64_t)ld16 * 2);
+  const int smem = (int)((gp ? 1 : 1 + gcap) * rowb);
   const bool conn = plan->connected == 1;
-  const void *kf = gp ? (conn ? (const void *)k_expand_pairs<true, true> : (const void *)k_expand_pairs<false, true>)
-                      : (conn ? (const void *)k_expand_pairs<true, false> : (const void *)k_expand_pairs<false, false>);
+  const void *kf = gp ? (two ? (conn ? (const void *)k_expand_pairs<true, true, 512> : (const void *)k_expand_pairs<false, true, 512>)
+                             : (conn ? (const void *)k_expand_pairs<true, true, 1024> : (const void *)k_expand_pairs<false, true, 1024>))
+                      : (conn ? (const void *)k_expand_pairs<true, false, 1024> : (const void *)k_expand_pairs<false, false, 1024>);
   EAR_CUDA_TRY(smem_attr(kf, smem));
   int32_t *counter = nullptr;
   EAR_CUDA_TRY(cudaMallocAsync((void **)&counter, sizeof(int32_t), st));
@@ -684,18 +695,17 @@ ear_status_t launch_pairs(const ear_plan_s *plan, const uint16_t *D16, int32_t l
   const XpView V{x->pd, x->rows, x->pstart, x->px, x->istart, x->tid2v};
   const double rows = row_end - row_begin;
   int se = prof_begin(prof_kind, st);
-  if (gp && conn)
-    EAR_LAUNCH((k_expand_pairs<true, true>), num_sms(), XP_NT, smem, st)(D16, ld16, nr, plan->desc, V, plan->n,
-                                                                          row_begin, row_end, out, ldo, gcap, counter);
-  else if (gp)
-    EAR_LAUNCH((k_expand_pairs<false, true>), num_sms(), XP_NT, smem, st)(D16, ld16, nr, plan->desc, V, plan->n,
-                                                                           row_begin, row_end, out, ldo, gcap, counter);
-  else if (conn)
-    EAR_LAUNCH((k_expand_pairs<true, false>), num_sms(), XP_NT, smem, st)(D16, ld16, nr, plan->desc, V, plan->n,
-                                                                           row_begin, row_end, out, ldo, gcap, counter);
-  else
-    EAR_LAUNCH((k_expand_pairs<false, false>), num_sms(), XP_NT, smem, st)(D16, ld16, nr, plan->desc, V, plan->n,
-                                                                            row_begin, row_end, out, ldo, gcap, counter);
+#define XP_GO(C, G, T, B)                                                                                      \
+  EAR_LAUNCH((k_expand_pairs<C, G, T>), (B) * num_sms(), T, smem, st)(D16, ld16, nr, plan->desc, V, plan->n, \
+                                                                       row_begin, row_end, out, ldo, gcap, counter)
+  if (gp && two) {
+    if (conn) XP_GO(true, true, 512, 2); else XP_GO(false, true, 512, 2);
+  } else if (gp) {
+    if (conn) XP_GO(true, true, 1024, 1); else XP_GO(false, true, 1024, 1);
+  } else {
+    if (conn) XP_GO(true, false, 1024, 1); else XP_GO(false, false, 1024, 1);
+  }
+#undef XP_GO
   // algorithmic bytes: the output, D read once (counted as the int32 D, as for the row-group kernel), the
   // descriptors
   prof_end(se, st, 4.0 * rows * plan->n + 16.0 * plan->n + 4.0 * (double)nr * nr * rows / plan->n);

@@ -242,11 +242,13 @@ def test_row_ranges_need_only_their_regions(pkg, rng_rows):
     assert ran
 
 
+@pytest.mark.parametrize("variant", ["0", "1", "2"])
 @pytest.mark.parametrize("case", ["cfg2", "corner", "cfg2_random"])
-def test_expansion_global_partners(pkg, case, monkeypatch):
-    """the pair-major expansion with only the item's row in shared memory and the partners' rows gathered
-    from global memory (cfg5's 120 KB rows need it), forced on small graphs by EAR_XP_GP=1"""
-    monkeypatch.setenv("EAR_XP_GP", "1")
+def test_expansion_variants(pkg, case, variant, monkeypatch):
+    """the pair-major expansion's three variants, forced by EAR_XP_GP: 0 the partners' rows staged beside the
+    item's, 1 only the item's row staged and the partners' gathered from global memory with two 512-thread
+    CTAs per SM (the default for cfg1-cfg4), 2 the same with one 1024-thread CTA (cfg5's 120 KB rows)"""
+    monkeypatch.setenv("EAR_XP_GP", variant)
     g = {"cfg2": lambda: gg.config("cfg2"), "corner": lambda: gg.corner_cases(17, n_target=1800),
          "cfg2_random": lambda: gg.config("cfg2", labels="random")}[case]()
     for flags in (pkg.FLAG_PART, pkg.FLAG_BCC):
