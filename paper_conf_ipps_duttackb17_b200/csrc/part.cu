@@ -1143,7 +1143,11 @@ ear_status_t part_build(const GView &gv, cudaStream_t st, ear_part_s **out) {
     EAR_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_partition, NT, 0));
     const int gc = (int)std::max<int64_t>(1, std::min<int64_t>(ceil_div(n, NT), (int64_t)per_sm * num_sms()));
     EAR_CUDA_TRY(dev_memset(flags, 0, 16 * sizeof(int32_t), st));
-    int32_t S = PSEED;
+    static const int32_t pseed = [] {   // lab knob: EAR_PSEED (seed spacing of the first Voronoi pass)
+      const char *e = getenv("EAR_PSEED");
+      return e ? std::max(2, atoi(e)) : PSEED;
+    }();
+    int32_t S = pseed;
     void *args[] = {(void *)&rowptr, (void *)&col, (void *)&cc, (void *)&n, (void *)&S, (void *)&lab[0], (void *)&lab[1],
                     (void *)&grp, (void *)&cnt, (void *)&flags};
     count_launch();
