@@ -1373,10 +1373,9 @@ ear_status_t part_solve(const GView &gv, ear_part_s *q, uint16_t *out, int64_t l
   EAR_CUDA_TRY(smem_attr((const void *)k_region_prod<true>, FINAL_SMEM));
   if (NB > 0) {
     EAR_LAUNCH(k_items, 1, 1024, 0, st)(q->roff, q->bcnt, q->K, NB, nullptr, items);
-    EAR_LAUNCH(k_region_prod<false>, (PR_MIN) * num_sms(), PR_NT, FINAL_SMEM, st)(LR, q->roff, q->bcnt, q->boff, q->perm, dB16,
-                                                                          NBp, NB, DBVt, NBp, q->reg, q->loc, cc,
-                                                                          q->rcomp, q->vrange, q->multi, items, q->K,
-                                                                          stats);
+    EAR_LAUNCH(k_region_prod<false>, PR_MIN * num_sms(), PR_NT, FINAL_SMEM, st)(
+        LR, q->roff, q->bcnt, q->boff, q->perm, dB16, NBp, NB, DBVt, NBp, q->reg, q->loc, cc, q->rcomp, q->vrange,
+        q->multi, items, q->K, stats);
     if (q->nbig > 0) {
       dim3 g1(NBp / MP_TC, q->nbig);
       EAR_LAUNCH(k_region_mp<false>, g1, MP_NT, 0, st)(LR, q->roff, q->bcnt, q->boff, q->perm, dB16, NBp, NBp, DBVt,
@@ -1392,9 +1391,9 @@ ear_status_t part_solve(const GView &gv, ear_part_s *q, uint16_t *out, int64_t l
   }
   tr.mark("product1+T");
   EAR_LAUNCH(k_items, 1, 1024, 0, st)(q->roff, q->bcnt, q->K, n, rneed, items);
-  EAR_LAUNCH(k_region_prod<true>, (PR_MIN) * num_sms(), PR_NT, FINAL_SMEM, st)(LR, q->roff, q->bcnt, q->boff, q->perm, DBV,
-                                                                       ldv, n, out, ldo, q->reg, q->loc, cc, q->rcomp,
-                                                                       q->vrange, q->multi, items, q->K, stats);
+  EAR_LAUNCH(k_region_prod<true>, PR_MIN * num_sms(), PR_NT, FINAL_SMEM, st)(
+      LR, q->roff, q->bcnt, q->boff, q->perm, DBV, ldv, n, out, ldo, q->reg, q->loc, cc, q->rcomp, q->vrange,
+      q->multi, items, q->K, stats);
   if (q->nbig > 0) {
     dim3 g2((unsigned)ceil_div(ldo, MP_TC), q->nbig);
     EAR_LAUNCH(k_region_mp<true>, g2, MP_NT, 0, st)(LR, q->roff, q->bcnt, q->boff, q->perm, DBVt, NBp, n, out, ldo,
