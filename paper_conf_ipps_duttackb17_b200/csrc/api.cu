@@ -316,15 +316,25 @@ static ear_status_t solve_rows(ear_plan_s *p, int32_t row_begin, int32_t row_end
   DKeep k;
   ear_status_t s = EAR_OK;
   LabTrace tr(st, -3);
-  if ((p->flags & EAR_FLAG_PART) && u16_ok && xp_applicable(p, st)) {
+  // the expansion's item lists: when the host can predict that they apply (no device check needed),
+  // they are enqueued from inside Phase II, while its last products run, so their host-side launch
+  // cost overlaps GPU work instead of delaying Phase II
+  bool part_xp = false;
+  bool xp_done = false;
+  const bool part_pred = (p->flags & EAR_FLAG_PART) && u16_ok && xp_predict(p);
+  if ((p->flags & EAR_FLAG_PART) && u16_ok && !part_pred) part_xp = xp_applicable(p, st), xp_done = true;
+  if (part_pred || part_xp) {
     tr.mark("solve: xp lists");
     // Phase II by regions straight into u16 rows; every rank computes all of D (a few ms) and expands
     // only its own output rows, so no exchange is needed
     k.ld16 = xp_row_stride(p);
     EAR_CUDA_TRY(cudaMallocAsync((void **)&k.D16, sizeof(uint16_t) * (size_t)p->n_reduced * k.ld16, st));
     bool applied = false;
-    s = part_rows(p, k.D16, k.ld16, nullptr, 0, 0, &applied, st, row_begin, row_end);
-    if (s != EAR_OK || !applied) {
+    s = part_rows(p, k.D16, k.ld16, nullptr, 0, 0, &applied, st, row_begin, row_end, [&] {
+      if (!xp_done) part_xp = xp_applicable(p, st), xp_done = true;
+    });
+    if (s == EAR_OK && !xp_done) part_xp = xp_applicable(p, st), xp_done = true;
+    if (s != EAR_OK || !applied || !part_xp) {
       cudaFreeAsync(k.D16, st);
       k.D16 = nullptr;
     }

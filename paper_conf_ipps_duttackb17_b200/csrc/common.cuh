@@ -4,6 +4,7 @@
 #include <cstdint>
 #include <cstdio>
 #include <cstdlib>
+#include <functional>
 #include <vector>
 #include <cuda_runtime.h>
 #include <nvtx3/nvToolsExt.h>
@@ -228,8 +229,11 @@ void bcc_free(ear_bcc_s *b, cudaStream_t stream);
 ear_status_t part_prepare(ear_plan_s *plan, cudaStream_t stream);
 // row_begin / row_end (D16 only): the caller's rows of G; D16 then holds only the rows Phase III stages
 // for them (the regions of their chain ends)
+// before_sync (optional): called once the last products are enqueued, before the final readback (host
+// work to overlap with them)
 ear_status_t part_rows(ear_plan_s *plan, uint16_t *D16, int64_t ld16, int32_t *D, int64_t ldd, int32_t Np,
-                       bool *applied, cudaStream_t stream, int32_t row_begin = 0, int32_t row_end = 0);
+                       bool *applied, cudaStream_t stream, int32_t row_begin = 0, int32_t row_end = 0,
+                       const std::function<void()> &before_sync = nullptr);
 void part_free(ear_part_s *q, cudaStream_t stream);
 // expand.cu
 ear_status_t expand(const ear_plan_s *plan, const int32_t *D, int64_t ldd, int32_t row_begin,
@@ -238,6 +242,8 @@ ear_status_t expand(const ear_plan_s *plan, const int32_t *D, int64_t ldd, int32
 // the path apsp_full takes when Phase II can hand over D16 (bcc_solve's u16 output)
 int32_t xp_row_stride(const ear_plan_s *plan);
 bool xp_applicable(ear_plan_s *plan, cudaStream_t stream);   // builds the item lists on first use
+bool xp_bounds_fit(const ear_plan_s *plan);
+bool xp_predict(const ear_plan_s *plan);   // xp_applicable's answer, known without building the lists
 ear_status_t expand_from16(const ear_plan_s *plan, const uint16_t *D16, int32_t ld16, int32_t row_begin,
                            int32_t row_end, int32_t *out, int64_t ldo, cudaStream_t stream, int prof_kind = PK_EXPAND);
 void xp_free(ear_xp_s *xp, cudaStream_t stream);

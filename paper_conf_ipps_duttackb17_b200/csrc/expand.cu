@@ -579,18 +579,21 @@ ear_status_t xp_build(ear_plan_s *p, cudaStream_t st) {
   ear_xp_s *x = new ear_xp_s;
   p->xp = x;
   const int32_t n = p->n, nr = p->n_reduced, nc = p->n_chain_vertices;
-  int32_t *bad = nullptr;
-  EAR_CUDA_TRY(cudaMallocAsync((void **)&bad, sizeof(int32_t), st));
-  EAR_CUDA_TRY(dev_memset(bad, 0, sizeof(int32_t), st));
-  EAR_LAUNCH(k_xp_flags, (int)std::min<int64_t>(ceil_div(n, 256), 148 * 16), 256, 0, st)(n, p->desc, bad);
-  int32_t h_bad = 1;
-  {
-    Readback rb(st);
-    EAR_CUDA_TRY(rb.get(&h_bad, bad, sizeof(int32_t)));
-    EAR_CUDA_TRY(rb.sync());
+  if (nr >= 0xFFFF) return EAR_OK;   // x->ok stays 0: the row-group kernel serves this plan
+  if (!xp_bounds_fit(p)) {   // the host bound is not enough: check the descriptors on the device
+    int32_t *bad = nullptr;
+    EAR_CUDA_TRY(cudaMallocAsync((void **)&bad, sizeof(int32_t), st));
+    EAR_CUDA_TRY(dev_memset(bad, 0, sizeof(int32_t), st));
+    EAR_LAUNCH(k_xp_flags, (int)std::min<int64_t>(ceil_div(n, 256), 148 * 16), 256, 0, st)(n, p->desc, bad);
+    int32_t h_bad = 1;
+    {
+      Readback rb(st);
+      EAR_CUDA_TRY(rb.get(&h_bad, bad, sizeof(int32_t)));
+      EAR_CUDA_TRY(rb.sync());
+    }
+    cudaFreeAsync(bad, st);
+    if (h_bad) return EAR_OK;
   }
-  cudaFreeAsync(bad, st);
-  if (h_bad || nr >= 0xFFFF) return EAR_OK;   // x->ok stays 0: the row-group kernel serves this plan
   auto g = [](int64_t k) { return (int)std::max<int64_t>(1, std::min<int64_t>(ceil_div(k, 256), 148 * 16)); };
   EAR_CUDA_TRY(cudaMallocAsync((void **)&x->pd, sizeof(uint2) * (size_t)std::max(n, 1), st));
   EAR_CUDA_TRY(cudaMallocAsync((void **)&x->tid2v, sizeof(int32_t) * (size_t)std::max(nr, 1), st));
@@ -763,6 +766,21 @@ ear_status_t expand_pairs(ear_plan_s *plan, const int32_t *D, int64_t ldd, int32
 }  // namespace
 
 int32_t xp_row_stride(const ear_plan_s *plan) { return (int32_t)round_up(std::max(plan->n_reduced, 1), 8); }
+
+// every chain offset fits 16 bits by the host's bound ((longest chain + 1) x heaviest edge) and every
+// terminal id too: the item lists can be built without a device check (no host round trip)
+bool xp_bounds_fit(const ear_plan_s *p) {
+  return p->n_reduced < 0xFFFF && ((int64_t)p->max_chain_len + 1) * (int64_t)std::max(p->max_weight, 0) <= 0xFFFF;
+}
+
+// xp_applicable's answer known on the host without building anything: the lists exist and apply, or
+// they will (no device check needed, the item's row fits a CTA)
+bool xp_predict(const ear_plan_s *plan) {
+  const char *env = getenv("EAR_EXPAND_PAIRS");
+  if (env && atoi(env) == 0) return false;
+  if (plan->xp) return plan->xp->ok != 0;
+  return xp_bounds_fit(plan) && xp_row_fits(plan->n_reduced);
+}
 
 bool xp_applicable(ear_plan_s *plan, cudaStream_t st) {
   const char *env = getenv("EAR_EXPAND_PAIRS");   // 0: the row-group kernel (A/B)

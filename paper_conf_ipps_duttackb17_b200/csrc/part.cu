@@ -1242,7 +1242,8 @@ ear_status_t part_prepare(ear_plan_s *p, cudaStream_t st) {
 // *applied = false when the route does not apply (too many regions, a region distance or a sum that
 // could reach 0xFFFF); nothing is written then.  Profiled (PK_PART / PK_PART_MP) at depth 0 only.
 ear_status_t part_solve(const GView &gv, ear_part_s *q, uint16_t *out, int64_t ldo, int depth, bool fw32,
-                        bool *applied, cudaStream_t st, const int32_t *rneed = nullptr) {
+                        bool *applied, cudaStream_t st, const int32_t *rneed = nullptr,
+                        const std::function<void()> &before_sync = nullptr) {
   *applied = false;
   const int32_t n = gv.n;
   // mostly tiny components (K near n): the (column blocks x regions) product grid would dominate
@@ -1400,6 +1401,7 @@ ear_status_t part_solve(const GView &gv, ear_part_s *q, uint16_t *out, int64_t l
                                                      q->reg, q->loc, cc, q->rcomp, q->multi, q->big, stats, rneed);
   }
   if (pm >= 0) prof_end(pm, st, (double)n * q->sum_rb + (double)NB * q->sum_rb);
+  if (before_sync) before_sync();   // the caller's host work overlaps the products
   int32_t h[4];
   EAR_TRY(rb1(h, stats, sizeof(h), st, "part_solve"));
   tr.mark("final product");
@@ -1411,7 +1413,7 @@ ear_status_t part_solve(const GView &gv, ear_part_s *q, uint16_t *out, int64_t l
 // Every row of D (reduced vertex order) as u16 (0xFFFF = INF, stride ld16 >= round_up(N_r, 8)), or
 // -- with D (int32, Np x Np, ldd) -- widened into it.  *applied = false when the route does not apply.
 ear_status_t part_rows(ear_plan_s *p, uint16_t *D16, int64_t ld16, int32_t *D, int64_t ldd, int32_t Np, bool *applied,
-                       cudaStream_t st, int32_t row_begin, int32_t row_end) {
+                       cudaStream_t st, int32_t row_begin, int32_t row_end, const std::function<void()> &before_sync) {
   NvtxRange nvtx_("ear: Phase II by regions");
   *applied = false;
   const int32_t n = p->n_reduced;
@@ -1445,7 +1447,7 @@ ear_status_t part_rows(ear_plan_s *p, uint16_t *D16, int64_t ld16, int32_t *D, i
     EAR_LAUNCH(k_need_rows, grid_n(row_end - row_begin), NT, 0, st)(p->desc, row_begin, row_end, need);
     EAR_LAUNCH(k_need_regions, grid_n(n), NT, 0, st)(need, p->part->reg, n, rneed);
   }
-  EAR_TRY(part_solve(gv, p->part, out, ldo, 0, (p->flags & EAR_FLAG_FW32) != 0, applied, st, rneed));
+  EAR_TRY(part_solve(gv, p->part, out, ldo, 0, (p->flags & EAR_FLAG_FW32) != 0, applied, st, rneed, before_sync));
   if (*applied && D) EAR_LAUNCH(k_widen, grid_n((int64_t)Np * Np), NT, 0, st)(out, ldo, n, D, ldd, Np);
   EAR_CUDA_TRY(cudaGetLastError());
   return EAR_OK;
