@@ -685,7 +685,8 @@ ear_status_t launch_pairs(const ear_plan_s *plan, const uint16_t *D16, int32_t l
   const int fv = force ? atoi(force) : -1;
   const bool two = 2 * (rowb + 4096) <= per_sm && fv != 2;
   const bool gp = fv >= 0 ? fv >= 1 : (two || xp_gcap(nr) < 1);
-  const int32_t gcap = gp ? XP_GMAX : xp_gcap(nr);
+  int32_t gcap = gp ? XP_GMAX : xp_gcap(nr);
+  if (const char *e = getenv("EAR_XP_GCAP")) gcap = std::max(1, std::min(gcap, atoi(e)));   // lab knob
   const int smem = (int)((gp ? 1 : 1 + gcap) * rowb);
   const bool conn = plan->connected == 1;
   const void *kf = gp ? (two ? (conn ? (const void *)k_expand_pairs<true, true, 512> : (const void *)k_expand_pairs<false, true, 512>)
