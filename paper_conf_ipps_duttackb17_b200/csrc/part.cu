@@ -996,6 +996,139 @@ __global__ void __launch_bounds__(256) k_fw64(uint16_t *M, int32_t N) {
   }
 }
 
+// The same 64-tile cooperative FW in int32 (one VIADDMNMX per min-plus, no cap): the boundary graphs
+// whose distances pass the u16 kernel's 0x7FFF cap (cfg5's deeper levels) -- instead of the 128-tile
+// TMA kernel, which is latency-bound at this size.  Thread (tr, tc) owns rows tr*4..+4, columns tc*4..+4.
+__device__ __forceinline__ void f64i_load(int32_t (*dst)[F64], const int32_t *M, int64_t ld, int ti, int tj) {
+  for (int e = threadIdx.x; e < F64 * F64 / 4; e += blockDim.x) {
+    const int r = e / 16, c4 = (e % 16) * 4;
+    *reinterpret_cast<int4 *>(&dst[r][c4]) = *reinterpret_cast<const int4 *>(M + (int64_t)(ti * F64 + r) * ld + tj * F64 + c4);
+  }
+}
+__device__ __forceinline__ void f64i_mp(const int32_t (*A)[F64], const int32_t (*B)[F64], int32_t c[4][4]) {
+  const int tr = threadIdx.x / 16, tc = threadIdx.x % 16;
+#pragma unroll 8
+  for (int m = 0; m < F64; ++m) {
+    const int4 av = *reinterpret_cast<const int4 *>(&A[m][tr * 4]);
+    const int4 bv = *reinterpret_cast<const int4 *>(&B[m][tc * 4]);
+    const int32_t a[4] = {av.x, av.y, av.z, av.w}, b[4] = {bv.x, bv.y, bv.z, bv.w};
+#pragma unroll
+    for (int q = 0; q < 4; ++q)
+#pragma unroll
+      for (int j = 0; j < 4; ++j) c[q][j] = __viaddmin_s32(a[q], b[j], c[q][j]);
+  }
+}
+__device__ __forceinline__ void f64i_store(int32_t *M, int64_t ld, int ti, int tj, const int32_t c[4][4], bool mirror) {
+  const int tr = threadIdx.x / 16, tc = threadIdx.x % 16;
+#pragma unroll
+  for (int q = 0; q < 4; ++q)
+    *reinterpret_cast<int4 *>(M + (int64_t)(ti * F64 + tr * 4 + q) * ld + tj * F64 + tc * 4) =
+        make_int4(c[q][0], c[q][1], c[q][2], c[q][3]);
+  if (mirror)
+#pragma unroll
+    for (int j = 0; j < 4; ++j)
+      *reinterpret_cast<int4 *>(M + (int64_t)(tj * F64 + tc * 4 + j) * ld + ti * F64 + tr * 4) =
+          make_int4(c[0][j], c[1][j], c[2][j], c[3][j]);
+}
+__global__ void __launch_bounds__(256) k_fw64i(int32_t *M, int32_t N) {
+  namespace cg = cooperative_groups;
+  cg::grid_group grid = cg::this_grid();
+  __shared__ __align__(16) int32_t As[F64][F64], Bs[F64][F64];
+  const int T = N / F64, tid = threadIdx.x, tr = tid / 16, tc = tid % 16;
+  auto close_tile = [&]() {   // As closed in place (an in-place step kk only reads row / column kk)
+    for (int kk = 0; kk < F64; ++kk) {
+      const int4 bv = *reinterpret_cast<const int4 *>(&As[kk][tc * 4]);
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        const int32_t a = As[tr * 4 + q][kk];
+        int4 cv = *reinterpret_cast<const int4 *>(&As[tr * 4 + q][tc * 4]);
+        cv.x = __viaddmin_s32(a, bv.x, cv.x);
+        cv.y = __viaddmin_s32(a, bv.y, cv.y);
+        cv.z = __viaddmin_s32(a, bv.z, cv.z);
+        cv.w = __viaddmin_s32(a, bv.w, cv.w);
+        *reinterpret_cast<int4 *>(&As[tr * 4 + q][tc * 4]) = cv;
+      }
+      __syncthreads();
+    }
+  };
+  auto store_tile = [&](int ti) {
+#pragma unroll
+    for (int q = 0; q < 4; ++q)
+      *reinterpret_cast<int4 *>(M + (int64_t)(ti * F64 + tr * 4 + q) * N + ti * F64 + tc * 4) =
+          *reinterpret_cast<const int4 *>(&As[tr * 4 + q][tc * 4]);
+  };
+  if (blockIdx.x == 0 && T > 0) {
+    f64i_load(As, M, N, 0, 0);
+    __syncthreads();
+    close_tile();
+    store_tile(0);
+  }
+  grid.sync();
+  for (int k = 0; k < T; ++k) {
+    if (blockIdx.x < T - 1) {
+      __syncthreads();
+      f64i_load(As, M, N, k, k);
+      __syncthreads();
+    }
+    for (int jt = blockIdx.x; jt < T - 1; jt += gridDim.x) {   // phase 2: pivot-row tiles, with transposes
+      const int j = jt < k ? jt : jt + 1;
+      __syncthreads();
+      f64i_load(Bs, M, N, k, j);
+      __syncthreads();
+      int32_t c[4][4];
+#pragma unroll
+      for (int q = 0; q < 4; ++q)
+#pragma unroll
+        for (int jj = 0; jj < 4; ++jj) c[q][jj] = Bs[tr * 4 + q][tc * 4 + jj];
+      f64i_mp(As, Bs, c);
+      f64i_store(M, N, k, j, c, true);
+    }
+    grid.sync();
+    if (blockIdx.x == 0 && k + 1 < T) {   // lookahead: the next pivot tile updated and closed by block 0
+      __syncthreads();
+      f64i_load(Bs, M, N, k, k + 1);
+      f64i_load(As, M, N, k + 1, k + 1);
+      __syncthreads();
+      int32_t c[4][4];
+#pragma unroll
+      for (int q = 0; q < 4; ++q)
+#pragma unroll
+        for (int jj = 0; jj < 4; ++jj) c[q][jj] = As[tr * 4 + q][tc * 4 + jj];
+      f64i_mp(Bs, Bs, c);
+      __syncthreads();
+#pragma unroll
+      for (int q = 0; q < 4; ++q) *reinterpret_cast<int4 *>(&As[tr * 4 + q][tc * 4]) = make_int4(c[q][0], c[q][1], c[q][2], c[q][3]);
+      __syncthreads();
+      close_tile();
+      store_tile(k + 1);
+    }
+    const int64_t nt = (int64_t)T * (T + 1) / 2;
+    const int64_t skip = (int64_t)(k + 1) * (k + 2) / 2 + (k + 1);
+    const int gb = gridDim.x > 1 ? (int)gridDim.x - 1 : 1;
+    for (int64_t e = gridDim.x > 1 ? blockIdx.x - 1 : 0; e < nt && (gridDim.x == 1 || blockIdx.x > 0); e += gb) {
+      if (k + 1 < T && e == skip) continue;
+      int i = (int)((sqrt(8.0 * (double)e + 1.0) - 1.0) / 2.0);
+      while ((int64_t)(i + 1) * (i + 2) / 2 <= e) ++i;
+      while ((int64_t)i * (i + 1) / 2 > e) --i;
+      const int jj = i, ii = (int)(e - (int64_t)i * (i + 1) / 2);
+      if (ii == k || jj == k) continue;
+      __syncthreads();
+      f64i_load(As, M, N, k, ii);
+      f64i_load(Bs, M, N, k, jj);
+      __syncthreads();
+      int32_t c[4][4];
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        const int4 x = *reinterpret_cast<const int4 *>(M + (int64_t)(ii * F64 + tr * 4 + q) * N + jj * F64 + tc * 4);
+        c[q][0] = x.x, c[q][1] = x.y, c[q][2] = x.z, c[q][3] = x.w;
+      }
+      f64i_mp(As, Bs, c);
+      f64i_store(M, N, ii, jj, c, ii != jj);
+    }
+    grid.sync();
+  }
+}
+
 __global__ void k_b16_fill(uint16_t *M, int32_t N) {
   const int64_t tot = (int64_t)N * N;
   for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < tot; e += (int64_t)gridDim.x * blockDim.x)
@@ -1342,6 +1475,31 @@ ear_status_t part_solve(const GView &gv, ear_part_s *q, uint16_t *out, int64_t l
       if (h_bad) EAR_CUDA_TRY(dev_memset(stats + 2, 0, sizeof(int32_t), st));   // the int32 FW redoes it
       done = !h_bad;
       tr.mark("dense boundary fw64");
+    }
+    if (!done && NB <= FW64_MAX) {   // dense, small, int32: the cooperative 64-tile FW without a cap
+      int32_t *M32 = nullptr;
+      const int32_t N64 = (int32_t)round_up(NB, F64);
+      if (!t.get(&M32, (size_t)N64 * N64)) {
+        set_error("part_solve: out of device memory");
+        return EAR_ENOMEM;
+      }
+      EAR_LAUNCH(k_bnd_fill, grid_n((int64_t)N64 * N64), NT, 0, st)(M32, N64);
+      EAR_LAUNCH(k_bnd_clique, q->K, NT, 0, st)(LR, q->bcnt, q->boff, M32, N64);
+      EAR_LAUNCH(k_bnd_cross, grid_n(NB), NT, 0, st)(gv.rowptr, gv.col, gv.w, q->bvert, NB, q->reg, q->gidx, M32, N64);
+      int per_sm = 0;
+      EAR_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_fw64i, 256, 0));
+      const int T = N64 / F64;
+      const int gfw = (int)std::max<int64_t>(1, std::min<int64_t>((int64_t)T * (T + 1) / 2, (int64_t)per_sm * num_sms()));
+      int32_t NN = N64;
+      void *args[] = {(void *)&M32, (void *)&NN};
+      count_launch();
+      if (cudaLaunchCooperativeKernel((const void *)k_fw64i, gfw, 256, args, 0, st) == cudaSuccess) {
+        EAR_LAUNCH(k_bnd_narrow, grid_n((int64_t)NB * NBp / 2), NT, 0, st)(M32, N64, NB, NBp, dB16, stats + 2);
+        done = true;
+      } else {
+        cudaGetLastError();
+      }
+      tr.mark("dense boundary fw64 int32");
     }
     if (!done) {   // dense: blocked FW over the boundary matrix
       int32_t *dB = nullptr, *labB = nullptr;
