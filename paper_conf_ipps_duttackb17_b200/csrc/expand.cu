@@ -56,6 +56,10 @@ __device__ __forceinline__ void st_cs_v4(int32_t *p, int4 v) {
                : "memory");
 }
 
+__device__ __forceinline__ void st_cs_s32(int32_t *p, int32_t v) {
+  asm volatile("st.global.cs.s32 [%0], %1;\n" ::"l"(p), "r"(v) : "memory");
+}
+
 __device__ __forceinline__ int32_t out_val(int32_t cp, int32_t rp, int32_t cq, int32_t rq) {
   // min(cp + rp, cq + rq, INF); every term < 2^31 (cp, cq < 2^30 by the EAR_EOVERFLOW check)
   return min(__viaddmin_s32(cq, rq, cp + rp), INF);
@@ -361,6 +365,15 @@ __global__ void k_xp_d16(const int32_t *__restrict__ D, int64_t ldd, int32_t nr,
   if (__syncthreads_or(b) && threadIdx.x == 0) atomicOr(bad, 1);
 }
 
+// L2 prefetch of one D16 row (bytes: a multiple of 16), spread over the 32 lanes of a warp in 4 KB pieces
+__device__ __forceinline__ void l2_prefetch_row(const uint16_t *row, int32_t bytes, int lane) {
+  for (int32_t o = lane * 4096; o < bytes; o += 32 * 4096) {
+    const int32_t sz = min(4096, bytes - o);
+    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;\n" ::"l"(reinterpret_cast<const char *>(row) + o), "r"(sz)
+                 : "memory");
+  }
+}
+
 __device__ __forceinline__ int32_t d16(const uint16_t *row, uint32_t t) {
   const uint32_t x = row[t];
   return x == 0xFFFFu ? INF : (int32_t)x;
@@ -389,11 +402,11 @@ __device__ __forceinline__ int32_t out_v(int32_t cp, int32_t rp, int32_t cq, int
 // per CTA two 512-thread CTAs share an SM (cfg4: 60 KB rows), so one's sweep building and row staging
 // overlap the other's column loop (measured 8.87 -> 8.47 ms on cfg4); rows too long for two per SM
 // (cfg5: 120 KB) run one 1024-thread CTA per SM.  !GP: the partners' rows staged beside the item's.
-template <bool CONN, bool GP, int NTT>
+template <bool CONN, bool GP, int NTT, bool LC = false>
 __global__ void __launch_bounds__(NTT, 1024 / NTT)
     k_expand_pairs(const uint16_t *__restrict__ D16, int32_t ldr, int32_t nr, const VDesc *__restrict__ desc,
                    const XpView X, int32_t n, int32_t rb, int32_t re, int32_t *__restrict__ out, int64_t ldo,
-                   int32_t gcap, int32_t *counter) {
+                   int32_t gcap, int32_t *counter, int32_t pf) {
   extern __shared__ __align__(16) uint16_t srow[];   // [1 + gcap][ldr]
   __shared__ int4 meta[XP_RMAX];                     // {c_sv, c_sx, slot, local output row}
   __shared__ int4 runs[XP_RMAX];                     // {slot, first meta row, end}: one per pair in the sweep
@@ -401,6 +414,7 @@ __global__ void __launch_bounds__(NTT, 1024 / NTT)
   __shared__ int32_t s_item, s_nrow, s_ns, s_pj, s_rj, s_nrun;
   const int tid = threadIdx.x;
   const uint32_t ldo_b = (uint32_t)(ldo * 4);
+  const int32_t row_bytes = ((nr + 7) / 8) * 16;
   for (;;) {
     if (tid == 0) s_item = atomicAdd(counter, 1);
     __syncthreads();
@@ -425,6 +439,7 @@ __global__ void __launch_bounds__(NTT, 1024 / NTT)
             if (slot < 0) {
               if (ns == gcap) break;
               if (lane == 0) slot_x[ns] = x;
+              if (GP && (pf & 1)) l2_prefetch_row(D16 + (int64_t)x * ldr, row_bytes, lane);
               __syncwarp();   // the other lanes read slot_x in the next partner's lookup
               slot = ++ns;
             }
@@ -486,6 +501,50 @@ __global__ void __launch_bounds__(NTT, 1024 / NTT)
                   reinterpret_cast<const uint4 *>(D16 + (int64_t)slot_x[k] * ldr)[i];
         loaded_v = true;
         __syncthreads();
+        if constexpr (LC) {
+          // lane-consecutive columns: lane l of warp w takes columns g*G + w*128 + l + 32*j (j < 4), so one
+          // gather instruction of a warp covers 32 adjacent columns, whose chain ends are close together
+          // (fewer distinct L1 lines / banks per gather than 4 columns per lane spread over 128)
+          constexpr int32_t G = NTT * 4;
+          const int32_t cw = (tid >> 5) * 128 + (tid & 31);
+          uint2 nd[4];
+#pragma unroll
+          for (int j = 0; j < 4; ++j) nd[j] = cw + 32 * j < n ? X.pd[cw + 32 * j] : make_uint2(0, 0);
+          for (int32_t c0 = cw; c0 < n; c0 += G) {
+            uint32_t pq[4], cc[4];
+#pragma unroll
+            for (int j = 0; j < 4; ++j) { pq[j] = nd[j].x; cc[j] = nd[j].y; }
+#pragma unroll
+            for (int j = 0; j < 4; ++j) nd[j] = c0 + G + 32 * j < n ? X.pd[c0 + G + 32 * j] : make_uint2(0, 0);
+            const bool full = c0 + 96 < n;
+            int32_t Rv[4];
+            r_of<CONN>(srow, pq, cc, Rv);
+            if (need_term) {
+              int32_t *o = reinterpret_cast<int32_t *>(reinterpret_cast<char *>(out) + (uint64_t)(uint32_t)(tv - rb) * ldo_b) + c0;
+#pragma unroll
+              for (int j = 0; j < 4; ++j)
+                if (full || c0 + 32 * j < n) st_cs_s32(o + 32 * j, Rv[j]);
+            }
+            for (int ru = 0; ru < nrun; ++ru) {
+              const int4 R = runs[ru];
+              int32_t Rx[4];
+              if (R.x == 0) {
+#pragma unroll
+                for (int j = 0; j < 4; ++j) Rx[j] = Rv[j];
+              } else {
+                r_of<CONN>(D16 + (int64_t)slot_x[R.x - 1] * ldr, pq, cc, Rx);
+              }
+              for (int r = R.y; r < R.z; ++r) {
+                const int4 m = meta[r];
+                int32_t *o = reinterpret_cast<int32_t *>(reinterpret_cast<char *>(out) + (uint64_t)(uint32_t)m.w * ldo_b) + c0;
+#pragma unroll
+                for (int j = 0; j < 4; ++j)
+                  if (full || c0 + 32 * j < n) st_cs_s32(o + 32 * j, out_v<CONN>(m.x, Rv[j], m.y, Rx[j]));
+              }
+            }
+          }
+          need_term = false;
+        } else {
         // descriptors of the next column group are loaded while the current one is computed and stored
         uint4 na = make_uint4(0, 0, 0, 0), nb4 = make_uint4(0, 0, 0, 0);
         if (tid * 4 + 4 <= n) {
@@ -542,6 +601,7 @@ __global__ void __launch_bounds__(NTT, 1024 / NTT)
           }
         }
         need_term = false;
+        }
       }
       __syncthreads();   // the next sweep rewrites meta, slot_x and the partner rows
       if (pj >= pe) break;
@@ -687,9 +747,15 @@ ear_status_t launch_pairs(const ear_plan_s *plan, const uint16_t *D16, int32_t l
   const bool gp = fv >= 0 ? fv >= 1 : (two || xp_gcap(nr) < 1);
   int32_t gcap = gp ? XP_GMAX : xp_gcap(nr);
   if (const char *e = getenv("EAR_XP_GCAP")) gcap = std::max(1, std::min(gcap, atoi(e)));   // lab knob
+  const char *le = getenv("EAR_XP_LC");   // lab knob: 0 = four adjacent columns per lane
+  const bool lc = gp && (le ? atoi(le) != 0 : true);
   const int smem = (int)((gp ? 1 : 1 + gcap) * rowb);
+  const char *pfe = getenv("EAR_XP_PF");
+  const int32_t pf = pfe ? atoi(pfe) : 0;   // lab knob: 1 = the partners' rows prefetched into L2
   const bool conn = plan->connected == 1;
-  const void *kf = gp ? (two ? (conn ? (const void *)k_expand_pairs<true, true, 512> : (const void *)k_expand_pairs<false, true, 512>)
+  const void *kf = lc ? (two ? (conn ? (const void *)k_expand_pairs<true, true, 512, true> : (const void *)k_expand_pairs<false, true, 512, true>)
+                              : (conn ? (const void *)k_expand_pairs<true, true, 1024, true> : (const void *)k_expand_pairs<false, true, 1024, true>))
+                 : gp ? (two ? (conn ? (const void *)k_expand_pairs<true, true, 512> : (const void *)k_expand_pairs<false, true, 512>)
                              : (conn ? (const void *)k_expand_pairs<true, true, 1024> : (const void *)k_expand_pairs<false, true, 1024>))
                       : (conn ? (const void *)k_expand_pairs<true, false, 1024> : (const void *)k_expand_pairs<false, false, 1024>);
   EAR_CUDA_TRY(smem_attr(kf, smem));
@@ -701,8 +767,15 @@ ear_status_t launch_pairs(const ear_plan_s *plan, const uint16_t *D16, int32_t l
   int se = prof_begin(prof_kind, st);
 #define XP_GO(C, G, T, B)                                                                                      \
   EAR_LAUNCH((k_expand_pairs<C, G, T>), (B) * num_sms(), T, smem, st)(D16, ld16, nr, plan->desc, V, plan->n, \
-                                                                       row_begin, row_end, out, ldo, gcap, counter)
-  if (gp && two) {
+                                                                       row_begin, row_end, out, ldo, gcap, counter, pf)
+#define XP_LC(C, T, B)                                                                                               \
+  EAR_LAUNCH((k_expand_pairs<C, true, T, true>), (B) * num_sms(), T, smem, st)(D16, ld16, nr, plan->desc, V, plan->n, \
+                                                                                row_begin, row_end, out, ldo, gcap, counter, pf)
+  if (lc && two) {
+    if (conn) XP_LC(true, 512, 2); else XP_LC(false, 512, 2);
+  } else if (lc) {
+    if (conn) XP_LC(true, 1024, 1); else XP_LC(false, 1024, 1);
+  } else if (gp && two) {
     if (conn) XP_GO(true, true, 512, 2); else XP_GO(false, true, 512, 2);
   } else if (gp) {
     if (conn) XP_GO(true, true, 1024, 1); else XP_GO(false, true, 1024, 1);
@@ -710,6 +783,7 @@ ear_status_t launch_pairs(const ear_plan_s *plan, const uint16_t *D16, int32_t l
     if (conn) XP_GO(true, false, 1024, 1); else XP_GO(false, false, 1024, 1);
   }
 #undef XP_GO
+#undef XP_LC
   // algorithmic bytes: the output, D read once (counted as the int32 D, as for the row-group kernel), the
   // descriptors
   prof_end(se, st, 4.0 * rows * plan->n + 16.0 * plan->n + 4.0 * (double)nr * nr * rows / plan->n);
