@@ -392,6 +392,19 @@ __device__ __forceinline__ void r_of(const uint16_t *row, const uint32_t pq[4], 
                                 d16(row, pq[j] & 0xFFFFu) + (int32_t)(cc[j] & 0xFFFFu)), INF);
   }
 }
+// r_of over a row in global memory, read through the non-coherent path (D16 is read-only here)
+template <bool CONN>
+__device__ __forceinline__ void r_of_g(const uint16_t *row, const uint32_t pq[4], const uint32_t cc[4], int32_t R[4]) {
+#pragma unroll
+  for (int j = 0; j < 4; ++j) {
+    const uint32_t a = __ldg(row + (pq[j] >> 16)), b = __ldg(row + (pq[j] & 0xFFFFu));
+    if (CONN)
+      R[j] = __viaddmin_s32((int32_t)a, (int32_t)(cc[j] >> 16), (int32_t)b + (int32_t)(cc[j] & 0xFFFFu));
+    else
+      R[j] = min(__viaddmin_s32(a == 0xFFFFu ? INF : (int32_t)a, (int32_t)(cc[j] >> 16),
+                                (b == 0xFFFFu ? INF : (int32_t)b) + (int32_t)(cc[j] & 0xFFFFu)), INF);
+  }
+}
 template <bool CONN>
 __device__ __forceinline__ int32_t out_v(int32_t cp, int32_t rp, int32_t cq, int32_t rq) {
   return CONN ? __viaddmin_s32(cq, rq, cp + rp) : out_val(cp, rp, cq, rq);
@@ -532,7 +545,9 @@ __global__ void __launch_bounds__(NTT, 1024 / NTT)
 #pragma unroll
                 for (int j = 0; j < 4; ++j) Rx[j] = Rv[j];
               } else {
-                r_of<CONN>(D16 + (int64_t)slot_x[R.x - 1] * ldr, pq, cc, Rx);
+                const uint16_t *prow = D16 + (int64_t)slot_x[R.x - 1] * ldr;
+                asm("" : "+l"(prow));   // one row pointer, not the row offset folded into every gather
+                r_of_g<CONN>(prow, pq, cc, Rx);
               }
               for (int r = R.y; r < R.z; ++r) {
                 const int4 m = meta[r];
