@@ -14,3 +14,5 @@ timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_re
 EAR_VERIFY_CFG5=1 EAR_VERIFY_OUT=gpurun_out/${T}_full_verify.jsonl timeout 1800 python -m pytest tests/test_full_verify_gpu.py -q -x -p no:cacheprovider -s -k part > gpurun_out/${T}_full_verify.txt 2>&1; echo "verify rc=$?"; tail -n 1 gpurun_out/${T}_full_verify.txt
 timeout 1500 python tools/time_routes.py --out gpurun_out/${T}_routes.jsonl > /dev/null 2>&1; echo "routes rc=$?"
 timeout 600 python tools/part_rank_timing.py cfg4 --out gpurun_out/${T}_part_rank_timing_cfg4.jsonl > /dev/null 2>&1; echo "rank timing rc=$?"
+for lab in morton random; do timeout 600 python tools/time_expand.py cfg4 --labels $lab --out gpurun_out/${T}_expand_labels.jsonl > /dev/null 2>&1; echo "expand cfg4 $lab rc=$?"; done
+timeout 600 python tools/time_expand.py cfg2 --labels random --out gpurun_out/${T}_expand_labels.jsonl > /dev/null 2>&1; echo "expand cfg2 random rc=$?"
