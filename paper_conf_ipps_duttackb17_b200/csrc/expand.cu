@@ -344,6 +344,25 @@ __global__ void k_xp_tid2v(int32_t n, const int32_t *tid, int32_t *tid2v) {
   for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x)
     if (tid[v] >= 0) tid2v[tid[v]] = (int32_t)v;
 }
+// Label locality for the choice of expansion variant: one warp per sampled window of 32 consecutive
+// columns; the window counts when its chain ends p_t (low half of pd.x) span fewer than XP_LOC_SPAN ids
+// (one L1 line of 64 u16 per 32 lanes on average at the limit).  Morton labels: cfg4 87 %, cfg2 95 %;
+// random labels: 0 %.
+constexpr int XP_LOC_SAMPLES = 1024, XP_LOC_SPAN = 1024;
+__global__ void k_xp_locality(const uint2 *__restrict__ pd, int32_t n, int32_t S, int32_t *count) {
+  const int lane = threadIdx.x & 31;
+  const int32_t w = (int32_t)((blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5);
+  if (w >= S) return;
+  const int32_t c = (int32_t)((int64_t)w * (n - 32) / S) + lane;
+  const int32_t x = (int32_t)(pd[c].x & 0xFFFFu);
+  int32_t lo = x, hi = x;
+  for (int o = 16; o; o >>= 1) {
+    lo = min(lo, __shfl_xor_sync(0xFFFFFFFFu, lo, o));
+    hi = max(hi, __shfl_xor_sync(0xFFFFFFFFu, hi, o));
+  }
+  if (lane == 0 && hi - lo < XP_LOC_SPAN) atomicAdd(count, 1);
+}
+
 // D (int32) -> u16 rows of stride ldr; a finite entry >= 0xFFFF sets *bad
 __global__ void k_xp_d16(const int32_t *__restrict__ D, int64_t ldd, int32_t nr, int32_t ldr, uint16_t *__restrict__ D16,
                          int32_t *bad) {
@@ -637,14 +656,24 @@ struct ear_xp_s {
   int32_t *px = nullptr;     // [npairs] the larger end (the partner)
   int32_t *istart = nullptr; // [N_r + 1] the pairs of each item (terminal = smaller end)
   int32_t *tid2v = nullptr;  // [N_r]
+  // label locality (k_xp_locality): sampled 32-column windows whose chain ends p_t span < XP_LOC_SPAN ids;
+  // written into pinned host memory, complete when loc_ev is
+  int32_t *loc_h = nullptr, *loc_d = nullptr, loc_samples = 0;
+  cudaEvent_t loc_ev = nullptr;
 };
 
 namespace ear {
 
 void xp_free(ear_xp_s *x, cudaStream_t st) {
   if (!x) return;
-  for (void *p : {(void *)x->pd, (void *)x->rows, (void *)x->pstart, (void *)x->px, (void *)x->istart, (void *)x->tid2v})
+  for (void *p : {(void *)x->pd, (void *)x->rows, (void *)x->pstart, (void *)x->px, (void *)x->istart, (void *)x->tid2v,
+                  (void *)x->loc_d})
     if (p) cudaFreeAsync(p, st);
+  if (x->loc_ev) {
+    cudaEventSynchronize(x->loc_ev);
+    cudaEventDestroy(x->loc_ev);
+  }
+  if (x->loc_h) cudaFreeHost(x->loc_h);
   delete x;
 }
 
@@ -675,6 +704,17 @@ ear_status_t xp_build(ear_plan_s *p, cudaStream_t st) {
   EAR_CUDA_TRY(cudaMallocAsync((void **)&x->istart, sizeof(int32_t) * ((size_t)nr + 1), st));
   EAR_LAUNCH(k_xp_desc, g(n), 256, 0, st)(n, p->desc, x->pd);
   EAR_LAUNCH(k_xp_tid2v, g(n), 256, 0, st)(n, p->tid, x->tid2v);
+  if (n >= 64 && cudaHostAlloc((void **)&x->loc_h, sizeof(int32_t), cudaHostAllocDefault) == cudaSuccess) {
+    x->loc_samples = (int32_t)std::min<int64_t>(XP_LOC_SAMPLES, n / 32);
+    EAR_CUDA_TRY(cudaMallocAsync((void **)&x->loc_d, sizeof(int32_t), st));
+    EAR_CUDA_TRY(dev_memset(x->loc_d, 0, sizeof(int32_t), st));
+    EAR_LAUNCH(k_xp_locality, ceil_div(x->loc_samples, 8), 256, 0, st)(x->pd, n, x->loc_samples, x->loc_d);
+    EAR_CUDA_TRY(cudaMemcpyAsync(x->loc_h, x->loc_d, sizeof(int32_t), cudaMemcpyDeviceToHost, st));
+    EAR_CUDA_TRY(cudaEventCreateWithFlags(&x->loc_ev, cudaEventDisableTiming));
+    EAR_CUDA_TRY(cudaEventRecord(x->loc_ev, st));
+  } else {
+    cudaGetLastError();
+  }
   x->nc = nc;
   uint64_t *k0 = nullptr, *k1 = nullptr;
   int32_t *v0 = nullptr, *head = nullptr, *hscan = nullptr, *pcount = nullptr;
@@ -759,7 +799,15 @@ ear_status_t launch_pairs(const ear_plan_s *plan, const uint16_t *D16, int32_t l
   const char *force = getenv("EAR_XP_GP");   // tests: 0 staged partners, 1 global (two CTAs/SM), 2 global (one)
   const int fv = force ? atoi(force) : -1;
   const bool two = 2 * (rowb + 4096) <= per_sm && fv != 2;
-  const bool gp = fv >= 0 ? fv >= 1 : (two || xp_gcap(nr) < 1);
+  // labels without locality (random: every gather its own sector) make the partners' gathers the
+  // bottleneck once D16 outgrows L2 (DRAM sectors): stage them instead when they fit (cfg4 random labels
+  // 19.6 -> 11.6 ms, Morton 9.2 vs 9.5; cfg2 random, D16 in L2: 0.55 global vs 0.66 staged)
+  bool local = true;
+  int l2 = 0;
+  EAR_CUDA_TRY(cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, dev));
+  if (x->loc_ev && (int64_t)nr * rowb > l2 && cudaEventSynchronize(x->loc_ev) == cudaSuccess)
+    local = 2 * *x->loc_h >= x->loc_samples;
+  const bool gp = fv >= 0 ? fv >= 1 : ((two && local) || xp_gcap(nr) < 1);
   int32_t gcap = gp ? XP_GMAX : xp_gcap(nr);
   if (const char *e = getenv("EAR_XP_GCAP")) gcap = std::max(1, std::min(gcap, atoi(e)));   // lab knob
   const char *le = getenv("EAR_XP_LC");   // lab knob: 0 = four adjacent columns per lane
