@@ -246,7 +246,8 @@ def test_row_ranges_need_only_their_regions(pkg, rng_rows):
 @pytest.mark.parametrize("case", ["cfg2", "corner", "cfg2_random"])
 def test_expansion_variants(pkg, case, variant, monkeypatch):
     """the pair-major expansion's three variants, forced by EAR_XP_GP: 0 the partners' rows staged beside the
-    item's, 1 only the item's row staged and the partners' gathered from global memory with two 512-thread
+    item's (chosen by default when the labels lack locality and D16 exceeds L2), 1 only the item's row
+    staged and the partners' gathered from global memory by lane-consecutive columns with two 512-thread
     CTAs per SM (the default for cfg1-cfg4), 2 the same with one 1024-thread CTA (cfg5's 120 KB rows)"""
     monkeypatch.setenv("EAR_XP_GP", variant)
     g = {"cfg2": lambda: gg.config("cfg2"), "corner": lambda: gg.corner_cases(17, n_target=1800),
