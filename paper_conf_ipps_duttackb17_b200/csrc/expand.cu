@@ -33,6 +33,8 @@
 #include <cub/cub.cuh>
 
 #include <algorithm>
+#include <mutex>
+#include <vector>
 #include <cstdlib>
 
 #include "common.cuh"
@@ -664,6 +666,43 @@ struct ear_xp_s {
 
 namespace ear {
 
+namespace {
+// 4-byte pinned host slots for the locality counts, from one portable pinned page allocated once per
+// process (a cudaHostAlloc / cudaFreeHost per plan would cost a synchronisation per apsp_full call)
+struct PinnedSlots {
+  std::mutex mu;
+  int32_t *base = nullptr;
+  std::vector<int> free;
+  bool failed = false;
+};
+PinnedSlots &pinned_slots() {
+  static PinnedSlots s;
+  return s;
+}
+int32_t *slot_get() {
+  PinnedSlots &s = pinned_slots();
+  std::lock_guard<std::mutex> lk(s.mu);
+  if (!s.base && !s.failed) {
+    if (cudaHostAlloc((void **)&s.base, 4096 * sizeof(int32_t), cudaHostAllocPortable) != cudaSuccess) {
+      cudaGetLastError();
+      s.base = nullptr;
+      s.failed = true;
+    } else {
+      for (int i = 4095; i >= 0; --i) s.free.push_back(i);
+    }
+  }
+  if (!s.base || s.free.empty()) return nullptr;
+  const int i = s.free.back();
+  s.free.pop_back();
+  return s.base + i;
+}
+void slot_put(int32_t *p) {
+  PinnedSlots &s = pinned_slots();
+  std::lock_guard<std::mutex> lk(s.mu);
+  s.free.push_back((int)(p - s.base));
+}
+}  // namespace
+
 void xp_free(ear_xp_s *x, cudaStream_t st) {
   if (!x) return;
   for (void *p : {(void *)x->pd, (void *)x->rows, (void *)x->pstart, (void *)x->px, (void *)x->istart, (void *)x->tid2v,
@@ -673,7 +712,7 @@ void xp_free(ear_xp_s *x, cudaStream_t st) {
     cudaEventSynchronize(x->loc_ev);
     cudaEventDestroy(x->loc_ev);
   }
-  if (x->loc_h) cudaFreeHost(x->loc_h);
+  if (x->loc_h) slot_put(x->loc_h);
   delete x;
 }
 
@@ -704,7 +743,7 @@ ear_status_t xp_build(ear_plan_s *p, cudaStream_t st) {
   EAR_CUDA_TRY(cudaMallocAsync((void **)&x->istart, sizeof(int32_t) * ((size_t)nr + 1), st));
   EAR_LAUNCH(k_xp_desc, g(n), 256, 0, st)(n, p->desc, x->pd);
   EAR_LAUNCH(k_xp_tid2v, g(n), 256, 0, st)(n, p->tid, x->tid2v);
-  if (n >= 64 && cudaHostAlloc((void **)&x->loc_h, sizeof(int32_t), cudaHostAllocDefault) == cudaSuccess) {
+  if (n >= 64 && (x->loc_h = slot_get()) != nullptr) {
     x->loc_samples = (int32_t)std::min<int64_t>(XP_LOC_SAMPLES, n / 32);
     EAR_CUDA_TRY(cudaMallocAsync((void **)&x->loc_d, sizeof(int32_t), st));
     EAR_CUDA_TRY(dev_memset(x->loc_d, 0, sizeof(int32_t), st));
@@ -712,8 +751,6 @@ ear_status_t xp_build(ear_plan_s *p, cudaStream_t st) {
     EAR_CUDA_TRY(cudaMemcpyAsync(x->loc_h, x->loc_d, sizeof(int32_t), cudaMemcpyDeviceToHost, st));
     EAR_CUDA_TRY(cudaEventCreateWithFlags(&x->loc_ev, cudaEventDisableTiming));
     EAR_CUDA_TRY(cudaEventRecord(x->loc_ev, st));
-  } else {
-    cudaGetLastError();
   }
   x->nc = nc;
   uint64_t *k0 = nullptr, *k1 = nullptr;
