@@ -996,6 +996,170 @@ __global__ void __launch_bounds__(256) k_fw64(uint16_t *M, int32_t N) {
   }
 }
 
+// k_fw64 with split barriers (the default; EAR_FW64_SPLIT=0 runs k_fw64): block 0 does the pivot-row tile (k, k+1) itself,
+// arrives at both barriers of round k at once and runs the update and closure of pivot k+1 while the other
+// blocks finish round k; they wait for the published pivot (flag) instead of a grid barrier after it.
+// Counters: bar[2k] (pivot row done), bar[2k+1] (round k done), bar[2T] = index of the last closed pivot + 1.
+__device__ __forceinline__ int ld_acquire_gpu(const int *p) {
+  int v;
+  asm volatile("ld.acquire.gpu.global.s32 %0, [%1];\n" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void sb_arrive(int *c) {
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    __threadfence();
+    atomicAdd(c, 1);
+  }
+}
+__device__ __forceinline__ void sb_wait(const int *c, int target) {
+  if (threadIdx.x == 0) {
+    while (ld_acquire_gpu(c) < target) __nanosleep(64);
+    __threadfence();
+  }
+  __syncthreads();
+}
+__device__ __forceinline__ void f64_close(uint16_t (*As)[F64]) {   // in place, one barrier per step
+  const int tr = threadIdx.x / 16, tc = threadIdx.x % 16;
+  for (int kk = 0; kk < F64; ++kk) {
+    const uint2 bv = *reinterpret_cast<const uint2 *>(&As[kk][tc * 4]);
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      const uint32_t a = dup16(As[tr * 4 + q][kk]);
+      uint2 cv = *reinterpret_cast<const uint2 *>(&As[tr * 4 + q][tc * 4]);
+      cv.x = __viaddmin_u16x2(a, bv.x, cv.x);
+      cv.y = __viaddmin_u16x2(a, bv.y, cv.y);
+      *reinterpret_cast<uint2 *>(&As[tr * 4 + q][tc * 4]) = cv;
+    }
+    __syncthreads();
+  }
+}
+__global__ void __launch_bounds__(256) k_fw64s(uint16_t *M, int32_t N, int *bar) {
+  __shared__ __align__(16) uint16_t As[F64][F64], Bs[F64][F64];
+  const int T = N / F64, tid = threadIdx.x, tr = tid / 16, tc = tid % 16;
+  const int G = gridDim.x, b = blockIdx.x;   // G >= 2 (the host checks)
+  int *piv = bar + 2 * T;
+  auto tile_to_smem = [&](uint16_t (*S)[F64], const uint32_t c[4][2]) {
+#pragma unroll
+    for (int q = 0; q < 4; ++q) *reinterpret_cast<uint2 *>(&S[tr * 4 + q][tc * 4]) = make_uint2(c[q][0], c[q][1]);
+  };
+  auto store_diag = [&](int ti) {
+#pragma unroll
+    for (int q = 0; q < 4; ++q)
+      *reinterpret_cast<uint2 *>(M + (int64_t)(ti * F64 + tr * 4 + q) * N + ti * F64 + tc * 4) =
+          *reinterpret_cast<const uint2 *>(&As[tr * 4 + q][tc * 4]);
+  };
+  if (b == 0) {
+    if (T > 0) {
+      f64_load(As, M, N, 0, 0);
+      __syncthreads();
+      f64_close(As);
+      store_diag(0);
+    }
+    __syncthreads();
+    if (tid == 0) {
+      __threadfence();
+      atomicExch(piv, 1);
+    }
+    for (int k = 0; k < T; ++k) {
+      if (k > 0) sb_wait(&bar[2 * (k - 1) + 1], G);   // round k-1 done everywhere
+      if (k + 1 < T) {
+        // As holds the closed pivot k; the pivot-row tile (k, k+1)
+        __syncthreads();
+        f64_load(Bs, M, N, k, k + 1);
+        __syncthreads();
+        uint32_t c[4][2];
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+          const uint2 x = *reinterpret_cast<const uint2 *>(&Bs[tr * 4 + q][tc * 4]);
+          c[q][0] = x.x, c[q][1] = x.y;
+        }
+        f64_mp(As, Bs, c);
+        f64_store(M, N, k, k + 1, c, true);
+        sb_arrive(&bar[2 * k]);
+        sb_arrive(&bar[2 * k + 1]);
+        // the next pivot: (k+1, k+1) = min(C, row(k,k+1)^T (x) row(k,k+1)), then closed
+        tile_to_smem(Bs, c);
+        f64_load(As, M, N, k + 1, k + 1);
+        __syncthreads();
+        uint32_t d[4][2];
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+          const uint2 x = *reinterpret_cast<const uint2 *>(&As[tr * 4 + q][tc * 4]);
+          d[q][0] = x.x, d[q][1] = x.y;
+        }
+        f64_mp(Bs, Bs, d);
+        __syncthreads();
+        tile_to_smem(As, d);
+        __syncthreads();
+        f64_close(As);
+        store_diag(k + 1);
+        __syncthreads();
+        if (tid == 0) {
+          __threadfence();
+          atomicExch(piv, k + 2);
+        }
+      } else {
+        sb_arrive(&bar[2 * k]);
+        sb_arrive(&bar[2 * k + 1]);
+      }
+    }
+    return;
+  }
+  const int gb = G - 1, bi = b - 1;
+  for (int k = 0; k < T; ++k) {
+    sb_wait(piv, k + 1);                              // pivot k closed
+    if (k > 0) sb_wait(&bar[2 * (k - 1) + 1], G);     // round k-1 done everywhere
+    // pivot-row tiles (k, j), j != k (and != k+1: block 0's)
+    const int nrow = k + 1 < T ? T - 2 : T - 1;
+    bool have_p = false;
+    for (int jt = bi; jt < nrow; jt += gb) {
+      int j = jt < k ? jt : jt + 1;   // skip k
+      if (k + 1 < T && j >= k + 1) ++j;   // skip k+1
+      __syncthreads();
+      if (!have_p) {
+        f64_load(As, M, N, k, k);
+        have_p = true;
+      }
+      f64_load(Bs, M, N, k, j);
+      __syncthreads();
+      uint32_t c[4][2];
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        const uint2 x = *reinterpret_cast<const uint2 *>(&Bs[tr * 4 + q][tc * 4]);
+        c[q][0] = x.x, c[q][1] = x.y;
+      }
+      f64_mp(As, Bs, c);
+      f64_store(M, N, k, j, c, true);
+    }
+    sb_arrive(&bar[2 * k]);
+    sb_wait(&bar[2 * k], G);
+    const int64_t nt = (int64_t)T * (T + 1) / 2;
+    const int64_t skip = (int64_t)(k + 1) * (k + 2) / 2 + (k + 1);   // (k+1, k+1): block 0's
+    for (int64_t e = bi; e < nt; e += gb) {
+      if (k + 1 < T && e == skip) continue;
+      int i = (int)((sqrt(8.0 * (double)e + 1.0) - 1.0) / 2.0);
+      while ((int64_t)(i + 1) * (i + 2) / 2 <= e) ++i;
+      while ((int64_t)i * (i + 1) / 2 > e) --i;
+      const int jj = i, ii = (int)(e - (int64_t)i * (i + 1) / 2);
+      if (ii == k || jj == k) continue;
+      __syncthreads();
+      f64_load(As, M, N, k, ii);
+      f64_load(Bs, M, N, k, jj);
+      __syncthreads();
+      uint32_t c[4][2];
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        const uint2 x = *reinterpret_cast<const uint2 *>(M + (int64_t)(ii * F64 + tr * 4 + q) * N + jj * F64 + tc * 4);
+        c[q][0] = x.x, c[q][1] = x.y;
+      }
+      f64_mp(As, Bs, c);
+      f64_store(M, N, ii, jj, c, ii != jj);
+    }
+    sb_arrive(&bar[2 * k + 1]);
+  }
+}
+
 // The same 64-tile cooperative FW in int32 (one VIADDMNMX per min-plus, no cap): the boundary graphs
 // whose distances pass the u16 kernel's 0x7FFF cap (cfg5's deeper levels) -- instead of the 128-tile
 // TMA kernel, which is latency-bound at this size.  Thread (tr, tc) owns rows tr*4..+4, columns tc*4..+4.
@@ -1459,13 +1623,29 @@ ear_status_t part_solve(const GView &gv, ear_part_s *q, uint16_t *out, int64_t l
       EAR_LAUNCH(k_b16_cross, grid_n(NB), NT, 0, st)(gv.rowptr, gv.col, gv.w, q->bvert, NB, q->reg, q->gidx, M, N64);
       int per_sm = 0;
       EAR_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_fw64, 256, 0));
+      {
+        int ps = 0;   // the split schedule's kernel must be co-resident with the same grid
+        EAR_CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&ps, k_fw64s, 256, 0));
+        per_sm = std::min(per_sm, ps);
+      }
       const int T = N64 / F64;
       const int gfw = (int)std::max<int64_t>(1, std::min<int64_t>((int64_t)T * (T + 1) / 2, (int64_t)per_sm * num_sms()));
       int32_t NN = N64;
       void *args[] = {(void *)&M, (void *)&NN};
       count_launch();
       int32_t h_bad = 1;
-      if (cudaLaunchCooperativeKernel((const void *)k_fw64, gfw, 256, args, 0, st) == cudaSuccess) {
+      const char *se = getenv("EAR_FW64_SPLIT");   // the split-barrier schedule (0: the grid-barrier kernel)
+      int *sbar = nullptr;
+      const bool split = (!se || atoi(se) != 0) && gfw >= 2 && t.get(&sbar, 2 * (size_t)T + 1);
+      cudaError_t le = cudaErrorUnknown;
+      if (split) {
+        EAR_CUDA_TRY(dev_memset(sbar, 0, sizeof(int) * (2 * (size_t)T + 1), st));
+        void *sargs[] = {(void *)&M, (void *)&NN, (void *)&sbar};
+        le = cudaLaunchCooperativeKernel((const void *)k_fw64s, gfw, 256, sargs, 0, st);
+      } else {
+        le = cudaLaunchCooperativeKernel((const void *)k_fw64, gfw, 256, args, 0, st);
+      }
+      if (le == cudaSuccess) {
         int32_t *st2 = stats + 2;
         EAR_LAUNCH(k_b16_narrow, grid_n((int64_t)NB * NBp), NT, 0, st)(M, N64, q->bvert, gv.cc, NB, NBp, dB16, st2, bad);
         EAR_TRY(rb1(&h_bad, bad, sizeof(int32_t), st, "part_solve"));

@@ -255,3 +255,19 @@ def test_expansion_variants(pkg, case, variant, monkeypatch):
     for flags in (pkg.FLAG_PART, pkg.FLAG_BCC):
         out, _ = run(pkg, g, flags=flags)
         exact(out.cpu().numpy(), oracle.apsp(g.n, g.src, g.dst, g.w), f"{case} flags={flags}")
+
+
+@pytest.mark.parametrize("split", ["0", "1"])
+@pytest.mark.parametrize("case", ["cfg2", "corner", "heavy20"])
+def test_boundary_fw_schedules(pkg, case, split, monkeypatch):
+    """the dense boundary FW (64-tile, one cooperative launch) under both schedules, forced by
+    EAR_FW64_SPLIT: 1 the split barriers (block 0 runs the next pivot while the others finish the round;
+    the default), 0 two grid barriers per round; heavy20: distances past the u16 cap (the int32 twin)"""
+    monkeypatch.setenv("EAR_FW64_SPLIT", split)
+    if case == "heavy20":
+        g0 = gg.torus(12, 12, 150, seed=3)
+        g = Graph(g0.n, g0.src, g0.dst, (g0.w.astype(np.int64) * 20).astype(np.int32))
+    else:
+        g = {"cfg2": lambda: gg.config("cfg2"), "corner": lambda: gg.corner_cases(5, n_target=1800)}[case]()
+    out, ran = run(pkg, g, flags=pkg.FLAG_PART | pkg.FLAG_SSSP)
+    exact(out.cpu().numpy(), oracle.apsp(g.n, g.src, g.dst, g.w), f"{case} split={split}")
